@@ -1,0 +1,255 @@
+"""Secure training / inference protocols, both parties simulated -- TEST INFRASTRUCTURE ONLY.
+
+Follows PAPER.md Sec. 4.3 "Detailed Design" (L201-L207): each layer runs a forward
+reconstruct (masking + opening) and a forward operation (Eq. 6/8), then a backward reconstruct
+and backward operation; B_i is the model, updated every step.  The fixed-point, truncation,
+activation-protocol, learning-rate and master-weight readings are DESIGN.md R3, R7, R9, R10,
+R13-R17.  The call-id layout (R11) is part of the parity contract with the CUDA path:
+
+    call_id = pair[63:56] | step[55:24] | layer[23:16] | op[15:8] | slot[7:0]
+
+ops: 0 forward matmul, 1 weight gradient, 2 input gradient, 3 ReLU MSB, 4 Eq. 9 MSB,
+6 Hadamard (slot 0 ReLU, 1 backprop DReLU, 2 Eq. 9), 7 share (slot 0 X, 1 Y, 2 init weight).
+
+All values are uint64 numpy arrays in Z_{2^64} (training is l = 64 only, R18).
+"""
+import numpy as np
+
+from . import core
+
+DATA_SEED = 0x50534D4C
+SHARE_SEED = DATA_SEED + 1
+DEALER_SEED = DATA_SEED + 2
+
+OP_FWD, OP_GRADW, OP_GRADIN, OP_RELU_MSB, OP_EQ9_MSB, OP_B2A, OP_HADAMARD, OP_SHARE = range(8)
+INIT_STEP = 0xFFFFFFFF
+
+F = 13            # fractional bits of activations / data / forward weights
+LR_SHIFT = 14     # eta / |B| = 2^-14  (eta = 2^-7, |B| = 128)
+MASTER = 27       # master-weight fractional bits m = F + LR_SHIFT (R14)
+L = 64
+MASK = np.uint64(0xFFFFFFFFFFFFFFFF)
+
+CNN_GEOM = dict(C=3, H=32, W=32, k=5, Cout=16, hidden=64, classes=10)
+
+
+def call_id(pair, step, layer, op, slot=0):
+    return ((pair & 0xFF) << 56) | ((step & 0xFFFFFFFF) << 24) | ((layer & 0xFF) << 16) \
+        | ((op & 0xFF) << 8) | (slot & 0xFF)
+
+
+def dims_of(task):
+    return {"linreg": [784, 1], "logreg": [784, 1], "mlp": [784, 128, 128, 10],
+            "cnn": [None, 12544, 64, 10]}[task]
+
+
+# ---------------------------------------------------------------------------------------------
+# client side: encode + share
+# ---------------------------------------------------------------------------------------------
+def share_batch(X, Y, step, pair=0):
+    x = core.encode(X, L, F)
+    y = core.encode(Y, L, F)
+    return (core.share(x, SHARE_SEED, call_id(pair, step, 0, OP_SHARE, 0)),
+            core.share(y, SHARE_SEED, call_id(pair, step, 0, OP_SHARE, 1)))
+
+
+def trunc_pair(x, d):
+    return core.truncate(x[0], 0, d), core.truncate(x[1], 1, d)
+
+
+def sub_pair(a, b):
+    return a[0] - b[0], a[1] - b[1]
+
+
+class Model:
+    """Both parties' weight shares: master (MASTER fractional bits) and forward copy (F bits)."""
+
+    def __init__(self, task, W_init):
+        self.task = task
+        self.Wm = []
+        for layer, W in enumerate(W_init):
+            w = core.encode(W, L, MASTER)
+            self.Wm.append(core.share(w, SHARE_SEED, call_id(0, INIT_STEP, layer, OP_SHARE, 2)))
+        self.W = [trunc_pair(wm, MASTER - F) for wm in self.Wm]
+
+    def decoded_master(self):
+        return [core.decode(core.reconstruct(*wm), L, MASTER) for wm in self.Wm]
+
+
+# ---------------------------------------------------------------------------------------------
+# dealer-aided building blocks (both parties)
+# ---------------------------------------------------------------------------------------------
+def _T(p):
+    return np.ascontiguousarray(p[0].T), np.ascontiguousarray(p[1].T)
+
+
+def matmul(A, B, pair, step, layer, op, trunc):
+    """Beaver product of two shared matrices with the triplet of call id (pair,step,layer,op)."""
+    M, K = A[0].shape
+    N = B[0].shape[1]
+    trip = core.triplet_gen(DEALER_SEED, call_id(pair, step, layer, op, 0), M, K, N, L)
+    return core.beaver_matmul(A, B, trip, trunc=trunc, l=L)
+
+
+def relu(z, pair, step, layer):
+    n = z[0].size
+    mat = core.msb_dealer(DEALER_SEED, call_id(pair, step, layer, OP_RELU_MSB, 0), n, L)
+    ht = core.hadamard_triplet_gen(DEALER_SEED, call_id(pair, step, layer, OP_HADAMARD, 0), n, L)
+    (r0, r1), (d0, d1) = core.secure_relu((z[0].reshape(-1), z[1].reshape(-1)), mat, ht, L)
+    s = z[0].shape
+    return (r0.reshape(s), r1.reshape(s)), (d0.reshape(s), d1.reshape(s))
+
+
+def eq9(z, pair, step, layer):
+    n = z[0].size
+    mat = core.msb_dealer(DEALER_SEED, call_id(pair, step, layer, OP_EQ9_MSB, 0), 2 * n, L)
+    ht = core.hadamard_triplet_gen(DEALER_SEED, call_id(pair, step, layer, OP_HADAMARD, 2), 2 * n, L)
+    return core.secure_eq9(z, mat, ht, L, F)
+
+
+def hadamard(a, b, pair, step, layer, slot):
+    n = a[0].size
+    ht = core.hadamard_triplet_gen(DEALER_SEED, call_id(pair, step, layer, OP_HADAMARD, slot), n, L)
+    c0, c1 = core.beaver_hadamard((a[0].reshape(-1), a[1].reshape(-1)),
+                                  (b[0].reshape(-1), b[1].reshape(-1)), ht, L)
+    return c0.reshape(a[0].shape), c1.reshape(a[0].shape)
+
+
+# --- CNN conv layer as im2col ring GEMM, masked in the un-expanded domain (R17) -------------
+def conv_triplet(pair, step, op, B, transpose):
+    """U over the raw input (B x C*H*W), V, Z = im2col(U).V (op 0) or im2col(U)^T.V (op 1)."""
+    g = CNN_GEOM
+    cid = call_id(pair, step, 0, op, 0)
+    nin = B * g["C"] * g["H"] * g["W"]
+    rows = B * (g["H"] - g["k"] + 1) * (g["W"] - g["k"] + 1)
+    kk = g["C"] * g["k"] * g["k"]
+    vshape = (rows, g["Cout"]) if transpose else (kk, g["Cout"])
+    U0 = core.prg(L, DEALER_SEED, core.tag("U0"), cid, nin).reshape(B, -1)
+    U1 = core.prg(L, DEALER_SEED, core.tag("U1"), cid, nin).reshape(B, -1)
+    nv = vshape[0] * vshape[1]
+    V0 = core.prg(L, DEALER_SEED, core.tag("V0"), cid, nv).reshape(vshape)
+    V1 = core.prg(L, DEALER_SEED, core.tag("V1"), cid, nv).reshape(vshape)
+    Ucol = core.im2col(U0 + U1, g["C"], g["H"], g["W"], g["k"])
+    Z = core.ring_matmul(np.ascontiguousarray(Ucol.T) if transpose else Ucol, V0 + V1)
+    Z0 = core.prg(L, DEALER_SEED, core.tag("Z0"), cid, Z.size).reshape(Z.shape)
+    return (U0, U1), (V0, V1), (Z0, Z - Z0)
+
+
+def conv_matmul(X, Bm, U, V, Z, transpose, trunc):
+    """C_i = i.E'.F + E'.V_i + U'_i.F + Z_i with E' = im2col(X - U) (^T), U'_i = im2col(U_i) (^T)."""
+    g = CNN_GEOM
+    col = lambda t: core.im2col(t, g["C"], g["H"], g["W"], g["k"])  # noqa: E731
+    tr = (lambda t: np.ascontiguousarray(t.T)) if transpose else (lambda t: t)  # noqa: E731
+    E = (X[0] - U[0]) + (X[1] - U[1])                       # Eq. 4 + Eq. 5 on the raw input
+    Fm = (Bm[0] - V[0]) + (Bm[1] - V[1])
+    Ec = tr(col(E))
+    EF = core.ring_matmul(Ec, Fm)
+    out = []
+    for i in range(2):
+        c = i * EF + core.ring_matmul(Ec, V[i]) + core.ring_matmul(tr(col(U[i])), Fm) + Z[i]
+        out.append(core.truncate(c, i, trunc) if trunc else c)
+    return tuple(out)
+
+
+# ---------------------------------------------------------------------------------------------
+# training step
+# ---------------------------------------------------------------------------------------------
+def forward_backward(model, Xs, Ys, step, pair=0):
+    """Returns (per-layer untruncated weight-gradient shares, prediction shares)."""
+    task = model.task
+    if task == "cnn":
+        return _cnn_forward_backward(model, Xs, Ys, step, pair)
+    nl = len(model.W)
+    acts = [Xs]
+    drelus = []
+    h = Xs
+    for layer in range(nl):
+        z = matmul(h, model.W[layer], pair, step, layer, OP_FWD, F)
+        if layer < nl - 1:
+            h, d = relu(z, pair, step, layer)
+            drelus.append(d)
+            acts.append(h)
+        elif task == "linreg":
+            h = z
+        else:
+            h = eq9(z, pair, step, layer)
+    yhat = h
+    delta = sub_pair(yhat, Ys)
+    grads = [None] * nl
+    for layer in range(nl - 1, -1, -1):
+        grads[layer] = matmul(_T(acts[layer]), delta, pair, step, layer, OP_GRADW, 0)
+        if layer > 0:
+            t = matmul(delta, _T(model.W[layer]), pair, step, layer, OP_GRADIN, F)
+            delta = hadamard(t, drelus[layer - 1], pair, step, layer - 1, 1)
+    return grads, yhat
+
+
+def _cnn_forward_backward(model, Xs, Ys, step, pair):
+    g = CNN_GEOM
+    B = Xs[0].shape[0]
+    U, V, Z = conv_triplet(pair, step, OP_FWD, B, transpose=False)
+    # forward conv: V for op 0 is the weight mask (75 x 16), Z = im2col(U) . V
+    zc = conv_matmul(Xs, model.W[0], U, V, Z, transpose=False, trunc=F)       # (B*784) x 16
+    h1, d1 = relu(zc, pair, step, 0)
+    h1 = (h1[0].reshape(B, -1), h1[1].reshape(B, -1))                         # B x 12544
+    z2 = matmul(h1, model.W[1], pair, step, 1, OP_FWD, F)
+    h2, d2 = relu(z2, pair, step, 1)
+    z3 = matmul(h2, model.W[2], pair, step, 2, OP_FWD, F)
+    yhat = eq9(z3, pair, step, 2)
+    delta = sub_pair(yhat, Ys)
+    grads = [None] * 3
+    grads[2] = matmul(_T(h2), delta, pair, step, 2, OP_GRADW, 0)
+    t = matmul(delta, _T(model.W[2]), pair, step, 2, OP_GRADIN, F)
+    delta = hadamard(t, d2, pair, step, 1, 1)
+    grads[1] = matmul(_T(h1), delta, pair, step, 1, OP_GRADW, 0)
+    t = matmul(delta, _T(model.W[1]), pair, step, 1, OP_GRADIN, F)
+    d1f = (d1[0].reshape(B, -1), d1[1].reshape(B, -1))
+    delta = hadamard(t, d1f, pair, step, 0, 1)
+    rows = B * (g["H"] - g["k"] + 1) * (g["W"] - g["k"] + 1)
+    delta = (delta[0].reshape(rows, g["Cout"]), delta[1].reshape(rows, g["Cout"]))
+    U, V, Z = conv_triplet(pair, step, OP_GRADW, B, transpose=True)
+    grads[0] = conv_matmul(Xs, delta, U, V, Z, transpose=True, trunc=0)
+    return grads, yhat
+
+
+def apply_update(model, grads, n_pairs=1):
+    """W^m_i -= trunc_i(gradW_i, F + log2(n_pairs)); W_i = trunc_i(W^m_i, MASTER - F)  (R14)."""
+    extra = int(np.log2(n_pairs))
+    assert (1 << extra) == n_pairs
+    for layer, g in enumerate(grads):
+        gt = trunc_pair(g, 26 + LR_SHIFT - MASTER + extra)
+        model.Wm[layer] = sub_pair(model.Wm[layer], gt)
+        model.W[layer] = trunc_pair(model.Wm[layer], MASTER - F)
+
+
+def train_step(model, X, Y, step, pair=0):
+    Xs, Ys = share_batch(X, Y, step, pair)
+    grads, yhat = forward_backward(model, Xs, Ys, step, pair)
+    apply_update(model, grads)
+    return yhat
+
+
+def infer(model, Xs, step, pair=0):
+    """Secure inference = the forward half."""
+    task = model.task
+    if task == "cnn":
+        B = Xs[0].shape[0]
+        U, V, Z = conv_triplet(pair, step, OP_FWD, B, transpose=False)
+        zc = conv_matmul(Xs, model.W[0], U, V, Z, transpose=False, trunc=F)
+        h, _ = relu(zc, pair, step, 0)
+        h = (h[0].reshape(B, -1), h[1].reshape(B, -1))
+        for layer in (1, 2):
+            z = matmul(h, model.W[layer], pair, step, layer, OP_FWD, F)
+            h = relu(z, pair, step, layer)[0] if layer == 1 else eq9(z, pair, step, layer)
+        return h
+    h = Xs
+    nl = len(model.W)
+    for layer in range(nl):
+        z = matmul(h, model.W[layer], pair, step, layer, OP_FWD, F)
+        if layer < nl - 1:
+            h = relu(z, pair, step, layer)[0]
+        elif task == "linreg":
+            h = z
+        else:
+            h = eq9(z, pair, step, layer)
+    return h

@@ -1,0 +1,431 @@
+/*
+ * psml_oracle.c -- CPU ORACLE for the ParSecureML hot path.  TEST INFRASTRUCTURE ONLY.
+ *
+ * Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline / --impl reference legs may
+ * load this library.  It shares no code, header, table or constant generator with the CUDA
+ * path under paper_conf_icpp_chenzzzz020_b200/ and never includes anything from it.
+ *
+ * What it is: a plain, slow, obviously-correct simulation of BOTH parties of the two-party
+ * Beaver-triplet protocol in the ring Z_{2^l} (values stored in uint64_t, reduced mod 2^l),
+ * written in the paper's order and notation:
+ *   PAPER.md L65-L78 (Sec. 2.2, Eqs. 1-6)  triplet multiplication, masking, opening, C_i
+ *   PAPER.md L164-L176 (Sec. 4.2, Eqs. 7-8) one-GEMM form (only used as a cross-check)
+ *   PAPER.md L178-L181 (Eq. 9)              piecewise-linear activation
+ *   PAPER.md L215-L228 (Eqs. 10-12)          delta + CSR compressed transmission
+ * plus the readings DESIGN.md lists where the paper is silent (ring, PRG, truncation, MSB
+ * protocol: DESIGN.md "Readings" R1..R18).
+ *
+ * Every loop is the textbook definition: no blocking, no fusion, no reordering.  The only
+ * concession to speed is `#pragma omp parallel for` over independent output rows/elements,
+ * which does not change any arithmetic (ring addition is exact).
+ *
+ * Parity pins (tests/test_oracle_*.py, marked "not gpu"):
+ *   chacha20 block      -> RFC 8439 Sec. 2.3.2 / 2.4.2 known-answer vectors
+ *   ring matmul         -> Python big-int brute force (independent arithmetic)
+ *   triplets / Beaver   -> closed forms Z0+Z1 = (U0+U1)(V0+V1), C0+C1 = A.B mod 2^l
+ *   truncation          -> SecureML Thm. 1 bound + stochastic-rounding statistics
+ *   MSB / ReLU / Eq. 9  -> exhaustive over all x in toy rings l = 8, 16 vs the sign bit
+ *   CSR codec           -> round trip and the 75%-zeros format rule
+ */
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+#include <math.h>
+
+#define EXPORT __attribute__((visibility("default")))
+
+static inline uint64_t ring_mask(int l) { return l >= 64 ? ~(uint64_t)0 : (((uint64_t)1 << l) - 1); }
+
+/* ------------------------------------------------------------------------------------------ */
+/* ChaCha20 block function, RFC 8439 Sec. 2.3 (R1: the PRG replacing MT19937 of       */
+/* PAPER.md L246).                                                                            */
+/* ------------------------------------------------------------------------------------------ */
+static inline uint32_t rotl32(uint32_t v, int c) { return (v << c) | (v >> (32 - c)); }
+
+#define QR(a, b, c, d)                 \
+    a += b; d ^= a; d = rotl32(d, 16); \
+    c += d; b ^= c; b = rotl32(b, 12); \
+    a += b; d ^= a; d = rotl32(d, 8);  \
+    c += d; b ^= c; b = rotl32(b, 7);
+
+EXPORT void or_chacha20_block(const uint32_t key[8], uint32_t counter, const uint32_t nonce[3],
+                              uint32_t out[16]) {
+    uint32_t s[16], x[16];
+    s[0] = 0x61707865u; s[1] = 0x3320646eu; s[2] = 0x79622d32u; s[3] = 0x6b206574u;
+    for (int i = 0; i < 8; ++i) s[4 + i] = key[i];
+    s[12] = counter;
+    s[13] = nonce[0]; s[14] = nonce[1]; s[15] = nonce[2];
+    for (int i = 0; i < 16; ++i) x[i] = s[i];
+    for (int r = 0; r < 10; ++r) {
+        QR(x[0], x[4], x[8], x[12]);
+        QR(x[1], x[5], x[9], x[13]);
+        QR(x[2], x[6], x[10], x[14]);
+        QR(x[3], x[7], x[11], x[15]);
+        QR(x[0], x[5], x[10], x[15]);
+        QR(x[1], x[6], x[11], x[12]);
+        QR(x[2], x[7], x[8], x[13]);
+        QR(x[3], x[4], x[9], x[14]);
+    }
+    for (int i = 0; i < 16; ++i) out[i] = x[i] + s[i];
+}
+
+/*
+ * PRG stream (R1): key = seed as 8 little-endian bytes || 24 zero bytes;
+ * nonce = 4-byte role tag || 8-byte call id, little endian; block counter = element / per_block.
+ * l > 32: element e = words (2j, 2j+1) of block e/8, j = e%8, little endian -> uint64.
+ * l <= 32: element e = word e%16 of block e/16.  Result reduced mod 2^l.
+ */
+EXPORT void or_prg(int l, uint64_t seed, uint32_t tag, uint64_t id, uint64_t offset, int64_t n,
+                   uint64_t *out) {
+    uint32_t key[8] = {(uint32_t)seed, (uint32_t)(seed >> 32), 0, 0, 0, 0, 0, 0};
+    uint32_t nonce[3] = {tag, (uint32_t)id, (uint32_t)(id >> 32)};
+    uint64_t m = ring_mask(l);
+    int per_block = l > 32 ? 8 : 16;
+#pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < n; ++i) {
+        uint64_t e = offset + (uint64_t)i;
+        uint32_t blk[16];
+        or_chacha20_block(key, (uint32_t)(e / per_block), nonce, blk);
+        int j = (int)(e % per_block);
+        uint64_t v = l > 32 ? ((uint64_t)blk[2 * j] | ((uint64_t)blk[2 * j + 1] << 32)) : blk[j];
+        out[i] = v & m;
+    }
+}
+
+/* ------------------------------------------------------------------------------------------ */
+/* Fixed-point encoding (R3; SecureML fixed point, not in PAPER.md which is FP32,     */
+/* L248/L260): v = round_half_even(x * 2^f) mod 2^l;  decode = signed(v) / 2^f.               */
+/* ------------------------------------------------------------------------------------------ */
+EXPORT void or_encode(int l, int f, const double *x, int64_t n, uint64_t *v) {
+    uint64_t m = ring_mask(l);
+    for (int64_t i = 0; i < n; ++i) {
+        long long r = llrint(ldexp(x[i], f)); /* default FP env: round half to even */
+        v[i] = (uint64_t)r & m;
+    }
+}
+
+EXPORT void or_decode(int l, int f, const uint64_t *v, int64_t n, double *x) {
+    uint64_t m = ring_mask(l);
+    for (int64_t i = 0; i < n; ++i) {
+        uint64_t u = v[i] & m;
+        int64_t s;
+        if (l < 64 && (u >> (l - 1)) & 1) s = (int64_t)(u - m - 1); /* u - 2^l */
+        else s = (int64_t)u;
+        x[i] = ldexp((double)s, -f);
+    }
+}
+
+/* ------------------------------------------------------------------------------------------ */
+/* Additive 2-party sharing, PAPER.md L65 ("randomly divide matrix A into A_0 and A_1") and    */
+/* L238 (A_0 random, A_1 by subtraction).  x_0 = PRG(seed, "SH", stream), x_1 = x - x_0.       */
+/* ------------------------------------------------------------------------------------------ */
+#define TAG(a, b, c, d) ((uint32_t)(uint8_t)(a) | ((uint32_t)(uint8_t)(b) << 8) | \
+                         ((uint32_t)(uint8_t)(c) << 16) | ((uint32_t)(uint8_t)(d) << 24))
+
+EXPORT void or_share(int l, uint64_t seed, uint64_t stream, const uint64_t *x, int64_t n,
+                     uint64_t *x0, uint64_t *x1) {
+    uint64_t m = ring_mask(l);
+    or_prg(l, seed, TAG('S', 'H', 0, 0), stream, 0, n, x0);
+    for (int64_t i = 0; i < n; ++i) x1[i] = (x[i] - x0[i]) & m;
+}
+
+EXPORT void or_reconstruct(int l, const uint64_t *x0, const uint64_t *x1, int64_t n, uint64_t *x) {
+    uint64_t m = ring_mask(l);
+    for (int64_t i = 0; i < n; ++i) x[i] = (x0[i] + x1[i]) & m;
+}
+
+/* Plain ring matmul C = A (MxK) . B (KxN) mod 2^l, row-major, schoolbook triple loop. */
+EXPORT void or_ring_matmul(int l, const uint64_t *A, const uint64_t *B, int64_t M, int64_t K,
+                           int64_t N, uint64_t *C) {
+    uint64_t m = ring_mask(l);
+#pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < M; ++i) {
+        for (int64_t j = 0; j < N; ++j) {
+            uint64_t acc = 0;
+            for (int64_t k = 0; k < K; ++k) acc += A[i * K + k] * B[k * N + j];
+            C[i * N + j] = acc & m;
+        }
+    }
+}
+
+/* ------------------------------------------------------------------------------------------ */
+/* Dealer (offline phase, Eqs. 2-3, Fig. 4): U, V random, Z = U x V,     */
+/* split into shares.  Reading R4: U_0,U_1,V_0,V_1,Z_0 from PRG streams, Z_1 = U V - Z_0.      */
+/* kind 0 = matrix triplet (U: MxK, V: KxN, Z: MxN); kind 1 = Hadamard (all n = M elements).   */
+/* ------------------------------------------------------------------------------------------ */
+EXPORT void or_triplet_gen(int l, uint64_t seed, uint64_t call_id, int64_t M, int64_t K, int64_t N,
+                           uint64_t *U0, uint64_t *U1, uint64_t *V0, uint64_t *V1, uint64_t *Z0,
+                           uint64_t *Z1) {
+    uint64_t m = ring_mask(l);
+    or_prg(l, seed, TAG('U', '0', 0, 0), call_id, 0, M * K, U0);
+    or_prg(l, seed, TAG('U', '1', 0, 0), call_id, 0, M * K, U1);
+    or_prg(l, seed, TAG('V', '0', 0, 0), call_id, 0, K * N, V0);
+    or_prg(l, seed, TAG('V', '1', 0, 0), call_id, 0, K * N, V1);
+    or_prg(l, seed, TAG('Z', '0', 0, 0), call_id, 0, M * N, Z0);
+    uint64_t *U = malloc(sizeof(uint64_t) * M * K), *V = malloc(sizeof(uint64_t) * K * N);
+    uint64_t *Z = malloc(sizeof(uint64_t) * M * N);
+    for (int64_t i = 0; i < M * K; ++i) U[i] = (U0[i] + U1[i]) & m;   /* Eq. 3 */
+    for (int64_t i = 0; i < K * N; ++i) V[i] = (V0[i] + V1[i]) & m;
+    or_ring_matmul(l, U, V, M, K, N, Z);                               /* Eq. 2 */
+    for (int64_t i = 0; i < M * N; ++i) Z1[i] = (Z[i] - Z0[i]) & m;   /* Eq. 3 */
+    free(U); free(V); free(Z);
+}
+
+EXPORT void or_hadamard_triplet_gen(int l, uint64_t seed, uint64_t call_id, int64_t n,
+                                    uint64_t *U0, uint64_t *U1, uint64_t *V0, uint64_t *V1,
+                                    uint64_t *Z0, uint64_t *Z1) {
+    uint64_t m = ring_mask(l);
+    or_prg(l, seed, TAG('U', '0', 0, 0), call_id, 0, n, U0);
+    or_prg(l, seed, TAG('U', '1', 0, 0), call_id, 0, n, U1);
+    or_prg(l, seed, TAG('V', '0', 0, 0), call_id, 0, n, V0);
+    or_prg(l, seed, TAG('V', '1', 0, 0), call_id, 0, n, V1);
+    or_prg(l, seed, TAG('Z', '0', 0, 0), call_id, 0, n, Z0);
+    for (int64_t i = 0; i < n; ++i) Z1[i] = (((U0[i] + U1[i]) * (V0[i] + V1[i])) - Z0[i]) & m;
+}
+
+/* ------------------------------------------------------------------------------------------ */
+/* Beaver matmul, Eqs. 4-6, simulated for both parties.                       */
+/*   Eq. 4: E_i = A_i - U_i, F_i = B_i - V_i        Eq. 5: E = E_0 + E_1, F = F_0 + F_1        */
+/*   form 0 (canonical, R2 = BASELINE north_star): C_i = i.E.F + E.V_i + U_i.F + Z_i  */
+/*   form 1 (paper Eq. 6):                                  C_i = (-i).E.F + A_i.F + E.B_i + Z_i */
+/* Then optional SecureML local truncation by `trunc` bits (R7).  Trace outputs are nullable.  */
+/* ------------------------------------------------------------------------------------------ */
+EXPORT void or_truncate(int l, int party, uint64_t *x, int64_t n, int d);
+
+EXPORT void or_beaver_matmul(int l, int form, const uint64_t *A0, const uint64_t *A1,
+                             const uint64_t *B0, const uint64_t *B1, const uint64_t *U0,
+                             const uint64_t *U1, const uint64_t *V0, const uint64_t *V1,
+                             const uint64_t *Z0, const uint64_t *Z1, int64_t M, int64_t K,
+                             int64_t N, int trunc, uint64_t *C0, uint64_t *C1,
+                             uint64_t *tE0, uint64_t *tE1, uint64_t *tE, uint64_t *tF0,
+                             uint64_t *tF1, uint64_t *tF) {
+    uint64_t m = ring_mask(l);
+    const uint64_t *A[2] = {A0, A1}, *B[2] = {B0, B1}, *U[2] = {U0, U1}, *V[2] = {V0, V1};
+    const uint64_t *Z[2] = {Z0, Z1};
+    uint64_t *C[2] = {C0, C1};
+    uint64_t *Ei[2], *Fi[2];
+    for (int i = 0; i < 2; ++i) { /* Eq. 4, party i */
+        Ei[i] = malloc(sizeof(uint64_t) * M * K);
+        Fi[i] = malloc(sizeof(uint64_t) * K * N);
+        for (int64_t t = 0; t < M * K; ++t) Ei[i][t] = (A[i][t] - U[i][t]) & m;
+        for (int64_t t = 0; t < K * N; ++t) Fi[i][t] = (B[i][t] - V[i][t]) & m;
+    }
+    uint64_t *E = malloc(sizeof(uint64_t) * M * K), *F = malloc(sizeof(uint64_t) * K * N);
+    for (int64_t t = 0; t < M * K; ++t) E[t] = (Ei[0][t] + Ei[1][t]) & m; /* Eq. 5 (opening) */
+    for (int64_t t = 0; t < K * N; ++t) F[t] = (Fi[0][t] + Fi[1][t]) & m;
+
+    uint64_t *EF = malloc(sizeof(uint64_t) * M * N), *T1 = malloc(sizeof(uint64_t) * M * N);
+    uint64_t *T2 = malloc(sizeof(uint64_t) * M * N);
+    or_ring_matmul(l, E, F, M, K, N, EF);
+    for (int i = 0; i < 2; ++i) {
+        if (form == 0) {
+            or_ring_matmul(l, E, V[i], M, K, N, T1);  /* E . V_i */
+            or_ring_matmul(l, U[i], F, M, K, N, T2);  /* U_i . F */
+            for (int64_t t = 0; t < M * N; ++t)
+                C[i][t] = ((uint64_t)i * EF[t] + T1[t] + T2[t] + Z[i][t]) & m;
+        } else {
+            or_ring_matmul(l, A[i], F, M, K, N, T1);  /* A_i . F */
+            or_ring_matmul(l, E, B[i], M, K, N, T2);  /* E . B_i */
+            for (int64_t t = 0; t < M * N; ++t)
+                C[i][t] = ((uint64_t)0 - (uint64_t)i * EF[t] + T1[t] + T2[t] + Z[i][t]) & m;
+        }
+        if (trunc > 0) or_truncate(l, i, C[i], M * N, trunc);
+    }
+    if (tE0) memcpy(tE0, Ei[0], sizeof(uint64_t) * M * K);
+    if (tE1) memcpy(tE1, Ei[1], sizeof(uint64_t) * M * K);
+    if (tE) memcpy(tE, E, sizeof(uint64_t) * M * K);
+    if (tF0) memcpy(tF0, Fi[0], sizeof(uint64_t) * K * N);
+    if (tF1) memcpy(tF1, Fi[1], sizeof(uint64_t) * K * N);
+    if (tF) memcpy(tF, F, sizeof(uint64_t) * K * N);
+    for (int i = 0; i < 2; ++i) { free(Ei[i]); free(Fi[i]); }
+    free(E); free(F); free(EF); free(T1); free(T2);
+}
+
+/* Beaver Hadamard (elementwise) product, same algebra with . replaced by (.) elementwise.     */
+EXPORT void or_beaver_hadamard(int l, const uint64_t *A0, const uint64_t *A1, const uint64_t *B0,
+                               const uint64_t *B1, const uint64_t *U0, const uint64_t *U1,
+                               const uint64_t *V0, const uint64_t *V1, const uint64_t *Z0,
+                               const uint64_t *Z1, int64_t n, uint64_t *C0, uint64_t *C1) {
+    uint64_t m = ring_mask(l);
+    for (int64_t t = 0; t < n; ++t) {
+        uint64_t e0 = A0[t] - U0[t], e1 = A1[t] - U1[t];
+        uint64_t f0 = B0[t] - V0[t], f1 = B1[t] - V1[t];
+        uint64_t e = (e0 + e1) & m, f = (f0 + f1) & m;
+        C0[t] = (0 * e * f + e * V0[t] + U0[t] * f + Z0[t]) & m;
+        C1[t] = (1 * e * f + e * V1[t] + U1[t] * f + Z1[t]) & m;
+    }
+}
+
+/* ------------------------------------------------------------------------------------------ */
+/* SecureML local share truncation (R7; not in PAPER.md): party 0: c >> d;                      */
+/* party 1: -((-c) >> d); logical shifts on l-bit unsigned values.                            */
+/* ------------------------------------------------------------------------------------------ */
+EXPORT void or_truncate(int l, int party, uint64_t *x, int64_t n, int d) {
+    uint64_t m = ring_mask(l);
+    if (d <= 0) return;
+    for (int64_t t = 0; t < n; ++t) {
+        uint64_t v = x[t] & m;
+        if (party == 0) x[t] = v >> d;
+        else x[t] = ((uint64_t)0 - ((((uint64_t)0 - v) & m) >> d)) & m;
+    }
+}
+
+/* ------------------------------------------------------------------------------------------ */
+/* Secure MSB / DReLU (R9; PAPER.md only says Eq. 9 is computed "in GPUs", L178).              */
+/* Dealer material per element e (all l-bit words):                                           */
+/*   AND index t = 0..2L-1 (L = log2 l): a_i, b_i, c_0 from PRG tags {'a','0'+i,t}, ...,        */
+/*   c_1 = ((a_0^a_1) & (b_0^b_1)) ^ c_0;                                                     */
+/*   daBit: rB_i = PRG('R','0'+i) & 1; rA_0 = PRG('R','A'); rA_1 = (rB_0 ^ rB_1) - rA_0.        */
+/* Material layout per party (uint64 words): [t][3][n] for (a,b,c) then rB[n], rA[n].           */
+/* ------------------------------------------------------------------------------------------ */
+static int log2_l(int l) { int L = 0; while ((1 << L) < l) ++L; return L; }
+
+EXPORT int64_t or_msb_material_words(int l, int64_t n) { return (int64_t)(2 * log2_l(l) * 3 + 2) * n; }
+
+EXPORT void or_msb_dealer(int l, uint64_t seed, uint64_t call_id, int64_t n, uint64_t *mat0,
+                          uint64_t *mat1) {
+    uint64_t m = ring_mask(l);
+    int L = log2_l(l);
+    uint64_t *mat[2] = {mat0, mat1};
+    for (int t = 0; t < 2 * L; ++t) {
+        for (int i = 0; i < 2; ++i) {
+            or_prg(l, seed, TAG('a', '0' + i, t, 0), call_id, 0, n, mat[i] + ((int64_t)t * 3 + 0) * n);
+            or_prg(l, seed, TAG('b', '0' + i, t, 0), call_id, 0, n, mat[i] + ((int64_t)t * 3 + 1) * n);
+        }
+        uint64_t *c0 = mat0 + ((int64_t)t * 3 + 2) * n, *c1 = mat1 + ((int64_t)t * 3 + 2) * n;
+        or_prg(l, seed, TAG('c', '0', t, 0), call_id, 0, n, c0);
+        for (int64_t e = 0; e < n; ++e) {
+            uint64_t a = mat0[((int64_t)t * 3 + 0) * n + e] ^ mat1[((int64_t)t * 3 + 0) * n + e];
+            uint64_t b = mat0[((int64_t)t * 3 + 1) * n + e] ^ mat1[((int64_t)t * 3 + 1) * n + e];
+            c1[e] = ((a & b) ^ c0[e]) & m;
+        }
+    }
+    int64_t off = (int64_t)2 * L * 3 * n;
+    or_prg(l, seed, TAG('R', '0', 0, 0), call_id, 0, n, mat0 + off);
+    or_prg(l, seed, TAG('R', '1', 0, 0), call_id, 0, n, mat1 + off);
+    for (int64_t e = 0; e < n; ++e) { mat0[off + e] &= 1; mat1[off + e] &= 1; }
+    or_prg(l, seed, TAG('R', 'A', 0, 0), call_id, 0, n, mat0 + off + n);
+    for (int64_t e = 0; e < n; ++e)
+        mat1[off + n + e] = ((mat0[off + e] ^ mat1[off + e]) - mat0[off + n + e]) & m;
+}
+
+/* One boolean Beaver AND for both parties on word vectors (GMW with a triplet):
+ * open e = x ^ a, f = y ^ b; z_i = (i ? e&f : 0) ^ (e & b_i) ^ (a_i & f) ^ c_i. */
+static void bool_and(int64_t n, const uint64_t *x0, const uint64_t *x1, const uint64_t *y0,
+                     const uint64_t *y1, const uint64_t *a0, const uint64_t *a1, const uint64_t *b0,
+                     const uint64_t *b1, const uint64_t *c0, const uint64_t *c1, uint64_t *z0,
+                     uint64_t *z1) {
+    for (int64_t t = 0; t < n; ++t) {
+        uint64_t e = (x0[t] ^ a0[t]) ^ (x1[t] ^ a1[t]);
+        uint64_t f = (y0[t] ^ b0[t]) ^ (y1[t] ^ b1[t]);
+        uint64_t r0 = (e & b0[t]) ^ (a0[t] & f) ^ c0[t];
+        uint64_t r1 = (e & f) ^ (e & b1[t]) ^ (a1[t] & f) ^ c1[t];
+        z0[t] = r0; z1[t] = r1;
+    }
+}
+
+/*
+ * MSB of x = x_0 + x_1 mod 2^l, Kogge-Stone carry prefix on boolean shares.
+ * P0 holds X0 := x_0 shared as (x_0, 0); P1 holds X1 := x_1 shared as (0, x_1).
+ * G = X0 & X1 (AND t=0); P = X0 ^ X1 (local).  For level j = 1..L, k = 2^(j-1):
+ *   G <- G ^ (P & (G << k))   (AND t = 2j-1)
+ *   P <- P & (P << k)         (AND t = 2j, skipped at j = L)
+ * msb = P_orig[l-1] ^ G[l-2].  Then B2A with the daBit: open c = msb ^ rB,
+ * [msb]^A_i = (i==0 ? c : 0) + (1 - 2c) rA_i.   Output: arithmetic shares of msb (0/1).
+ * Optional output: boolean shares of msb (bit 0 of a word).
+ */
+EXPORT void or_secure_msb(int l, const uint64_t *x0, const uint64_t *x1, int64_t n,
+                          const uint64_t *mat0, const uint64_t *mat1, uint64_t *msbA0,
+                          uint64_t *msbA1, uint64_t *msbB0, uint64_t *msbB1) {
+    uint64_t m = ring_mask(l);
+    int L = log2_l(l);
+    size_t sz = sizeof(uint64_t) * n;
+    uint64_t *X0s0 = calloc(n, sizeof(uint64_t)), *X0s1 = calloc(n, sizeof(uint64_t));
+    uint64_t *X1s0 = calloc(n, sizeof(uint64_t)), *X1s1 = calloc(n, sizeof(uint64_t));
+    uint64_t *G0 = malloc(sz), *G1 = malloc(sz), *P0 = malloc(sz), *P1 = malloc(sz);
+    uint64_t *S0 = malloc(sz), *S1 = malloc(sz), *T0 = malloc(sz), *T1 = malloc(sz);
+    for (int64_t t = 0; t < n; ++t) { X0s0[t] = x0[t] & m; X1s1[t] = x1[t] & m; }
+#define MAT(i, tt, w) ((i) == 0 ? mat0 : mat1) + ((int64_t)(tt) * 3 + (w)) * n
+    bool_and(n, X0s0, X0s1, X1s0, X1s1, MAT(0, 0, 0), MAT(1, 0, 0), MAT(0, 0, 1), MAT(1, 0, 1),
+             MAT(0, 0, 2), MAT(1, 0, 2), G0, G1);
+    for (int64_t t = 0; t < n; ++t) { P0[t] = X0s0[t] ^ X1s0[t]; P1[t] = X0s1[t] ^ X1s1[t]; }
+    for (int j = 1; j <= L; ++j) {
+        int k = 1 << (j - 1);
+        for (int64_t t = 0; t < n; ++t) { S0[t] = (G0[t] << k) & m; S1[t] = (G1[t] << k) & m; }
+        bool_and(n, P0, P1, S0, S1, MAT(0, 2 * j - 1, 0), MAT(1, 2 * j - 1, 0), MAT(0, 2 * j - 1, 1),
+                 MAT(1, 2 * j - 1, 1), MAT(0, 2 * j - 1, 2), MAT(1, 2 * j - 1, 2), T0, T1);
+        if (j < L) {
+            for (int64_t t = 0; t < n; ++t) { S0[t] = (P0[t] << k) & m; S1[t] = (P1[t] << k) & m; }
+            uint64_t *Q0 = malloc(sz), *Q1 = malloc(sz);
+            bool_and(n, P0, P1, S0, S1, MAT(0, 2 * j, 0), MAT(1, 2 * j, 0), MAT(0, 2 * j, 1),
+                     MAT(1, 2 * j, 1), MAT(0, 2 * j, 2), MAT(1, 2 * j, 2), Q0, Q1);
+            memcpy(P0, Q0, sz); memcpy(P1, Q1, sz);
+            free(Q0); free(Q1);
+        }
+        for (int64_t t = 0; t < n; ++t) { G0[t] ^= T0[t]; G1[t] ^= T1[t]; }
+    }
+#undef MAT
+    int64_t off = (int64_t)2 * L * 3 * n;
+    for (int64_t t = 0; t < n; ++t) {
+        uint64_t b0 = ((X0s0[t] >> (l - 1)) & 1) ^ ((G0[t] >> (l - 2)) & 1); /* P_orig share 0 = x_0 */
+        uint64_t b1 = ((X1s1[t] >> (l - 1)) & 1) ^ ((G1[t] >> (l - 2)) & 1); /* P_orig share 1 = x_1 */
+        if (msbB0) msbB0[t] = b0;
+        if (msbB1) msbB1[t] = b1;
+        uint64_t c = (b0 ^ mat0[off + t]) ^ (b1 ^ mat1[off + t]); /* B2A opening */
+        uint64_t s = (1 - 2 * c) & m;
+        msbA0[t] = (c + s * mat0[off + n + t]) & m;
+        msbA1[t] = (s * mat1[off + n + t]) & m;
+    }
+    free(X0s0); free(X0s1); free(X1s0); free(X1s1);
+    free(G0); free(G1); free(P0); free(P1); free(S0); free(S1); free(T0); free(T1);
+}
+
+/* ------------------------------------------------------------------------------------------ */
+/* CSR codec of PAPER.md L228 (compressed transmission of the inter-epoch delta, Eqs. 10-12).  */
+/* Delta = cur - prev (mod 2^l), viewed as rows x cols.  CSR iff 4*nnz <= rows*cols (>= 75%   */
+/* zeros), else dense.  Returns nnz; row_ptr[rows+1], col_idx[nnz], vals[nnz] filled for CSR. */
+/* ------------------------------------------------------------------------------------------ */
+EXPORT int64_t or_delta_csr_encode(int l, const uint64_t *cur, const uint64_t *prev, int64_t rows,
+                                   int64_t cols, int32_t *is_csr, int32_t *row_ptr,
+                                   int32_t *col_idx, uint64_t *vals, uint64_t *dense) {
+    uint64_t m = ring_mask(l);
+    int64_t nnz = 0;
+    for (int64_t t = 0; t < rows * cols; ++t) nnz += ((cur[t] - prev[t]) & m) != 0;
+    *is_csr = (4 * nnz <= rows * cols);
+    if (*is_csr) {
+        int64_t k = 0;
+        row_ptr[0] = 0;
+        for (int64_t r = 0; r < rows; ++r) {
+            for (int64_t c = 0; c < cols; ++c) {
+                uint64_t d = (cur[r * cols + c] - prev[r * cols + c]) & m;
+                if (d) { col_idx[k] = (int32_t)c; vals[k] = d; ++k; }
+            }
+            row_ptr[r + 1] = (int32_t)k;
+        }
+    } else {
+        for (int64_t t = 0; t < rows * cols; ++t) dense[t] = (cur[t] - prev[t]) & m;
+    }
+    return nnz;
+}
+
+EXPORT void or_delta_csr_apply(int l, int64_t rows, int64_t cols, int32_t is_csr,
+                               const int32_t *row_ptr, const int32_t *col_idx, const uint64_t *vals,
+                               const uint64_t *dense, uint64_t *target) {
+    uint64_t m = ring_mask(l);
+    if (is_csr) {
+        for (int64_t r = 0; r < rows; ++r)
+            for (int32_t k = row_ptr[r]; k < row_ptr[r + 1]; ++k)
+                target[r * cols + col_idx[k]] = (target[r * cols + col_idx[k]] + vals[k]) & m;
+    } else {
+        for (int64_t t = 0; t < rows * cols; ++t) target[t] = (target[t] + dense[t]) & m;
+    }
+}
+
+EXPORT int or_num_threads(void) {
+#ifdef _OPENMP
+    extern int omp_get_max_threads(void);
+    return omp_get_max_threads();
+#else
+    return 1;
+#endif
+}

@@ -1,0 +1,142 @@
+"""Seeded synthetic plaintext inputs shared by the oracle, the tests and bench.py.
+
+This module holds NONE of the method's arithmetic (no encoding, sharing, ring or protocol
+step): it only produces float64 plaintext data, labels and initial weights with the shapes and
+value distributions of the paper's workloads:
+
+  * MNIST-shaped rows (28x28 pixels 0..255): 784 features in [0, 1], about 81%
+    exact zeros, non-zeros U(0, 1] (MNIST's ~19% ink density), scaled by 1/255 semantics.
+  * CIFAR-10-shaped rows (3x32x32): 3072 dense U(0, 1) features.
+  * labels from fixed random teachers (linear, thresholded linear, 784-128-128-10 ReLU MLP,
+    5x5/16-channel conv net), one-hot for the 10-class tasks.
+
+Every 128-row block b is drawn from its own generator ``default_rng([seed, kind, b])``, so any
+row range is reproducible without generating the rows before it (the bench only materialises
+the steps it times; the parity tests slice the same rows).
+"""
+import functools
+
+import numpy as np
+
+DATA_SEED = 0x50534D4C          # "PSML"
+INIT_SEED = DATA_SEED + 3
+TEACHER_SEED = DATA_SEED + 4
+BLOCK = 128
+
+MNIST_FEATURES = 784
+CIFAR_SHAPE = (3, 32, 32)
+CIFAR_FEATURES = 3 * 32 * 32
+
+_KIND = {"mnist": 1, "cifar": 2}
+
+
+def _block_rows(kind, b, seed):
+    rng = np.random.default_rng([seed, _KIND[kind], b])
+    if kind == "mnist":
+        x = rng.random((BLOCK, MNIST_FEATURES))
+        keep = rng.random((BLOCK, MNIST_FEATURES)) < 0.19
+        return np.where(keep, 1.0 - x, 0.0)                 # non-zeros in (0, 1]
+    return rng.random((BLOCK, CIFAR_FEATURES))
+
+
+def rows(kind, start, count, seed=DATA_SEED):
+    """Rows [start, start+count) of the synthetic dataset `kind` ('mnist' | 'cifar')."""
+    if count <= 0:
+        width = MNIST_FEATURES if kind == "mnist" else CIFAR_FEATURES
+        return np.zeros((0, width))
+    b0, b1 = start // BLOCK, (start + count - 1) // BLOCK
+    blocks = np.concatenate([_block_rows(kind, b, seed) for b in range(b0, b1 + 1)], axis=0)
+    off = start - b0 * BLOCK
+    return blocks[off:off + count]
+
+
+# ---------------------------------------------------------------------------------------------
+# teachers (label generators)
+# ---------------------------------------------------------------------------------------------
+def linear_teacher(d=MNIST_FEATURES, seed=TEACHER_SEED):
+    return np.random.default_rng([seed, 1]).uniform(-0.05, 0.05, size=(d, 1))
+
+
+@functools.lru_cache(maxsize=None)
+def logistic_threshold(seed=TEACHER_SEED):
+    """Median of X w* over the first 8192 MNIST-shaped rows (fixed, data-independent of step)."""
+    w = linear_teacher(seed=seed)
+    return float(np.median(rows("mnist", 0, 8192) @ w))
+
+
+def mlp_teacher(dims=(784, 128, 128, 10), seed=TEACHER_SEED):
+    rng = np.random.default_rng([seed, 3])
+    return [rng.normal(0.0, 1.0, size=(a, b)) / np.sqrt(a) for a, b in zip(dims[:-1], dims[1:])]
+
+
+def cnn_teacher(seed=TEACHER_SEED, cout=16, k=5, hidden=64, classes=10):
+    rng = np.random.default_rng([seed, 4])
+    c = CIFAR_SHAPE[0]
+    oh = CIFAR_SHAPE[1] - k + 1
+    return [rng.normal(0.0, 1.0, size=(c * k * k, cout)) / np.sqrt(c * k * k),
+            rng.normal(0.0, 1.0, size=(oh * oh * cout, hidden)) / np.sqrt(oh * oh * cout),
+            rng.normal(0.0, 1.0, size=(hidden, classes)) / np.sqrt(hidden)]
+
+
+def _patches(X, k=5):
+    """(B, 3072) -> (B*28*28, 75) patch matrix for the teacher conv (label generation only)."""
+    B = X.shape[0]
+    c, h, w = CIFAR_SHAPE
+    oh, ow = h - k + 1, w - k + 1
+    X4 = X.reshape(B, c, h, w)
+    out = np.empty((B, oh, ow, c, k, k))
+    for ky in range(k):
+        for kx in range(k):
+            out[:, :, :, :, ky, kx] = X4[:, :, ky:ky + oh, kx:kx + ow].transpose(0, 2, 3, 1)
+    return out.reshape(B * oh * ow, c * k * k)
+
+
+def _one_hot(scores):
+    y = np.zeros_like(scores)
+    y[np.arange(scores.shape[0]), np.argmax(scores, axis=1)] = 1.0
+    return y
+
+
+def labels(task, X):
+    relu = lambda t: np.maximum(t, 0.0)   # noqa: E731  (teacher nets only)
+    if task == "linreg":
+        return X @ linear_teacher()
+    if task == "logreg":
+        return (X @ linear_teacher() > logistic_threshold()).astype(np.float64)
+    if task == "mlp":
+        W = mlp_teacher()
+        return _one_hot(relu(relu(X @ W[0]) @ W[1]) @ W[2])
+    if task == "cnn":
+        Wc, W1, W2 = cnn_teacher()
+        h = relu(_patches(X) @ Wc).reshape(X.shape[0], -1)
+        return _one_hot(relu(h @ W1) @ W2)
+    raise ValueError(task)
+
+
+TASK_DATA = {"linreg": "mnist", "logreg": "mnist", "mlp": "mnist", "cnn": "cifar"}
+TASK_ROWS = {"mnist": 60000, "cifar": 50000}
+
+
+def batch(task, step, batch_size=BLOCK, pair=0, n_pairs=1, seed=DATA_SEED):
+    """Minibatch `step` of `task` for data-parallel pair `pair` of `n_pairs` (weak scaling:
+    each pair gets its own `batch_size` rows).  Returns float64 (X, Y)."""
+    kind = TASK_DATA[task]
+    start = ((step * n_pairs + pair) * batch_size) % (TASK_ROWS[kind] - batch_size + 1)
+    X = rows(kind, start, batch_size, seed)
+    return X, labels(task, X)
+
+
+def init_weights(task, dims=None, seed=INIT_SEED):
+    """Initial plaintext weights (R13): zeros for linear/logistic regression,
+    U(+-1/sqrt(fan_in)) for the MLP and CNN."""
+    if task in ("linreg", "logreg"):
+        return [np.zeros((MNIST_FEATURES, 1))]
+    if task == "mlp":
+        dims = dims or (784, 128, 128, 10)
+        shapes = list(zip(dims[:-1], dims[1:]))
+    elif task == "cnn":
+        shapes = [(75, 16), (12544, 64), (64, 10)]
+    else:
+        raise ValueError(task)
+    rng = np.random.default_rng([seed, 7])
+    return [rng.uniform(-1.0, 1.0, size=s) / np.sqrt(s[0]) for s in shapes]

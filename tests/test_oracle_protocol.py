@@ -1,0 +1,72 @@
+"""Pins of the oracle's protocol layer (not gpu): golden worked examples, training vs fp64."""
+import glob
+import json
+import os
+
+import numpy as np
+import pytest
+
+import synth
+from oracle import plain
+from oracle import protocol as P
+
+GOLDEN = sorted(glob.glob(os.path.join(os.path.dirname(__file__), "golden", "beaver_*.json")))
+
+
+def _a(x):
+    return np.array(x, dtype=np.uint64)
+
+
+@pytest.mark.parametrize("path", GOLDEN, ids=[os.path.basename(p) for p in GOLDEN])
+def test_oracle_matches_golden(orc, path):
+    d = json.load(open(path))
+    l = d["l"]
+    trip = tuple(_a(d[k]) for k in ("U0", "U1", "V0", "V1", "Z0", "Z1"))
+    A = (_a(d["A0"]), _a(d["A1"]))
+    B = (_a(d["B0"]), _a(d["B1"]))
+    (C0, C1), tr = orc.beaver_matmul(A, B, trip, l=l, trace=True)
+    for k in ("E0", "E1", "E", "F0", "F1", "F"):
+        assert tr[k].tolist() == d[k], k
+    assert C0.tolist() == d["C0"] and C1.tolist() == d["C1"]
+    P0, P1 = orc.beaver_matmul(A, B, trip, form=1, l=l)
+    assert P0.tolist() == d["P0"] and P1.tolist() == d["P1"]
+    T0, T1 = orc.beaver_matmul(A, B, trip, trunc=d["trunc"], l=l)
+    assert T0.tolist() == d["T0"] and T1.tolist() == d["T1"]
+    assert orc.reconstruct(C0, C1, l).tolist() == d["AB"]
+
+
+def test_call_id_layout():
+    assert P.call_id(0xAB, 0x12345678, 0xCD, 0xEF, 0x99) == 0xAB12345678CDEF99
+    assert P.call_id(1, 0, 0, 0, 0) == 1 << 56
+
+
+def _train(task, steps):
+    Wi = synth.init_weights(task)
+    m, pm = P.Model(task, Wi), plain.PlainModel(task, Wi)
+    for s in range(steps):
+        X, Y = synth.batch(task, s)
+        P.train_step(m, X, Y, s)
+        pm.step(X, Y)
+    return max(np.abs(a - b).max() for a, b in zip(m.decoded_master(), pm.W))
+
+
+@pytest.mark.parametrize("task,steps,tol_log2", [("linreg", 60, -16), ("logreg", 60, -16),
+                                                  ("mlp", 8, -15)])
+def test_oracle_training_tracks_fp64(task, steps, tol_log2):
+    """Decoded master weights vs plaintext fp64 SGD (BASELINE north_star pin, shortened run;
+    the full-epoch 2^-12 check runs on the GPU path in tests/test_gpu_training.py)."""
+    err = _train(task, steps)
+    assert err < 2.0 ** tol_log2, np.log2(err)
+
+
+def test_oracle_inference_matches_plaintext_forward():
+    task = "mlp"
+    Wi = synth.init_weights(task)
+    m, pm = P.Model(task, Wi), plain.PlainModel(task, Wi)
+    X, Y = synth.batch(task, 3)
+    Xs, _ = P.share_batch(X, Y, 3)
+    yh = P.infer(m, Xs, step=1000)
+    from oracle import core
+    got = core.decode(core.reconstruct(*yh))
+    want = pm.forward(plain.q(X, P.F))[2]
+    assert np.abs(got - want).max() < 2.0 ** -9
