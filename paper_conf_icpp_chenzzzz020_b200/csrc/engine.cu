@@ -1,0 +1,426 @@
+// engine.cu -- the C ABI of include/psml.h: context, client/dealer calls, secure ops.
+// Models / training live in model.cu.
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <string>
+
+#include "engine.h"
+
+namespace psml {
+
+static thread_local std::string g_err;
+std::atomic<uint64_t> g_launches{0};
+
+void set_error(const std::string &msg) { g_err = msg; }
+psml_status fail(psml_status st, const std::string &msg) {
+    g_err = msg;
+    return st;
+}
+
+int current_sm_count() {
+    int dev = 0, sms = 148;
+    if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    return sms;
+}
+
+psml_status check_ring(psml_ring r) {
+    if (r.l != 32 && r.l != 64) return fail(PSML_ERR_INVALID, "ring.l must be 32 or 64");
+    if (r.frac_bits < 0 || r.frac_bits >= r.l) return fail(PSML_ERR_INVALID, "ring.frac_bits out of range");
+    return PSML_OK;
+}
+
+psml_status check_ptrs(std::initializer_list<const void *> ps) {
+    for (const void *p : ps) {
+        if (p == nullptr) return fail(PSML_ERR_INVALID, "null device pointer");
+        if (!aligned16(p)) return fail(PSML_ERR_ALIGN, "pointer not 16-byte aligned");
+    }
+    return PSML_OK;
+}
+
+psml_status Ctx::ensure_ws(size_t bytes) {
+    if (bytes <= ws_bytes) return PSML_OK;
+    if (ws) {
+        PSML_CUDA_TRY(cudaDeviceSynchronize());
+        PSML_CUDA_TRY(cudaFree(ws));
+        ws = nullptr;
+        ws_bytes = 0;
+    }
+    size_t want = std::max(bytes, (size_t)1 << 20);
+    if (cudaMalloc(&ws, want) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(PSML_ERR_NOMEM, "workspace allocation of " + std::to_string(want) + " bytes failed");
+    }
+    ws_bytes = want;
+    return PSML_OK;
+}
+
+}  // namespace psml
+
+using namespace psml;
+
+// ABI definitions: C linkage and default visibility come from include/psml.h.
+
+int32_t psml_abi_version(void) { return PSML_ABI_VERSION; }
+const char *psml_last_error(void) { return g_err.c_str(); }
+uint64_t psml_kernel_launch_count(void) { return g_launches.load(); }
+
+psml_status psml_device_info(int32_t *sm_count, int32_t *cc_major, int32_t *cc_minor) {
+    int dev = 0, n = 0;
+    if (cudaGetDeviceCount(&n) != cudaSuccess || n == 0) {
+        cudaGetLastError();
+        return fail(PSML_ERR_UNSUPPORTED, "no CUDA device visible");
+    }
+    PSML_CUDA_TRY(cudaGetDevice(&dev));
+    int a = 0, b = 0, c = 0;
+    PSML_CUDA_TRY(cudaDeviceGetAttribute(&a, cudaDevAttrMultiProcessorCount, dev));
+    PSML_CUDA_TRY(cudaDeviceGetAttribute(&b, cudaDevAttrComputeCapabilityMajor, dev));
+    PSML_CUDA_TRY(cudaDeviceGetAttribute(&c, cudaDevAttrComputeCapabilityMinor, dev));
+    if (sm_count) *sm_count = a;
+    if (cc_major) *cc_major = b;
+    if (cc_minor) *cc_minor = c;
+    return PSML_OK;
+}
+
+psml_status psml_ctx_create(psml_ring ring, int32_t gemm_backend, psml_ctx *out) {
+    PSML_TRY(check_ring(ring));
+    if (!out) return fail(PSML_ERR_INVALID, "out is null");
+    if (gemm_backend < 0 || gemm_backend > 2) return fail(PSML_ERR_INVALID, "gemm_backend must be 0, 1 or 2");
+    int32_t sms = 0, maj = 0, mnr = 0;
+    PSML_TRY(psml_device_info(&sms, &maj, &mnr));
+    if (gemm_backend == 2 && !(maj == 10 && mnr == 0))
+        return fail(PSML_ERR_UNSUPPORTED, "tcgen05 backend needs an sm_100 device");
+    Ctx *c = new Ctx();
+    c->ring = ring;
+    c->backend = gemm_backend;
+    c->sm_count = sms;
+    c->tc_ok = (maj == 10 && mnr == 0);
+    *out = reinterpret_cast<psml_ctx>(c);
+    return PSML_OK;
+}
+
+psml_status psml_ctx_destroy(psml_ctx ctx) {
+    if (!ctx) return PSML_OK;
+    Ctx *c = reinterpret_cast<Ctx *>(ctx);
+    if (c->ws) {
+        cudaDeviceSynchronize();
+        cudaFree(c->ws);
+    }
+    delete c;
+    return PSML_OK;
+}
+
+// ------------------------------------------------------------------------------------------------
+// client side
+// ------------------------------------------------------------------------------------------------
+psml_status psml_prg_fill(psml_ring ring, uint64_t seed, uint32_t tag, uint64_t call_id, uint64_t offset,
+                          int64_t n, void *out, psml_stream stream) {
+    PSML_TRY(check_ring(ring));
+    if (n < 0) return fail(PSML_ERR_SHAPE, "n < 0");
+    if (n == 0) return PSML_OK;
+    PSML_TRY(check_ptrs({out}));
+    cudaStream_t s = (cudaStream_t)stream;
+    PrgKey k = make_key(seed, tag, call_id);
+    const int64_t nblk = n / (ring.l == 64 ? 8 : 16) + 2;
+    if (ring.l == 64) prg_kernel<uint64_t, 0><<<grid_for(nblk, 256), 256, 0, s>>>(k, offset, n, (uint64_t *)out, nullptr, nullptr);
+    else prg_kernel<uint32_t, 0><<<grid_for(nblk, 256), 256, 0, s>>>(k, offset, n, (uint32_t *)out, nullptr, nullptr);
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
+psml_status psml_encode(psml_ring ring, const double *x, int64_t n, void *v, psml_stream stream) {
+    PSML_TRY(check_ring(ring));
+    if (n < 0) return fail(PSML_ERR_SHAPE, "n < 0");
+    if (n == 0) return PSML_OK;
+    PSML_TRY(check_ptrs({x, v}));
+    cudaStream_t s = (cudaStream_t)stream;
+    if (ring.l == 64) encode_kernel<uint64_t><<<grid_for(n, 256), 256, 0, s>>>(x, n, ring.frac_bits, (uint64_t *)v);
+    else encode_kernel<uint32_t><<<grid_for(n, 256), 256, 0, s>>>(x, n, ring.frac_bits, (uint32_t *)v);
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
+psml_status psml_decode(psml_ring ring, const void *v, int64_t n, double *x, psml_stream stream) {
+    PSML_TRY(check_ring(ring));
+    if (n < 0) return fail(PSML_ERR_SHAPE, "n < 0");
+    if (n == 0) return PSML_OK;
+    PSML_TRY(check_ptrs({x, v}));
+    cudaStream_t s = (cudaStream_t)stream;
+    if (ring.l == 64) decode_kernel<uint64_t><<<grid_for(n, 256), 256, 0, s>>>((const uint64_t *)v, n, ring.frac_bits, x);
+    else decode_kernel<uint32_t><<<grid_for(n, 256), 256, 0, s>>>((const uint32_t *)v, n, ring.frac_bits, x);
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
+psml_status psml_share(psml_ring ring, uint64_t seed, uint64_t stream_id, const void *x, int64_t n, void *x0,
+                       void *x1, psml_stream stream) {
+    PSML_TRY(check_ring(ring));
+    if (n < 0) return fail(PSML_ERR_SHAPE, "n < 0");
+    if (n == 0) return PSML_OK;
+    PSML_TRY(check_ptrs({x, x0, x1}));
+    if (x == x0 || x == x1 || x0 == x1) return fail(PSML_ERR_INVALID, "share outputs must not alias the input");
+    cudaStream_t s = (cudaStream_t)stream;
+    PrgKey k = make_key(seed, TAG_SH, stream_id);
+    const int64_t nblk = n / (ring.l == 64 ? 8 : 16) + 2;
+    if (ring.l == 64)
+        prg_kernel<uint64_t, 1><<<grid_for(nblk, 256), 256, 0, s>>>(k, 0, n, (uint64_t *)x0, (const uint64_t *)x, (uint64_t *)x1);
+    else
+        prg_kernel<uint32_t, 1><<<grid_for(nblk, 256), 256, 0, s>>>(k, 0, n, (uint32_t *)x0, (const uint32_t *)x, (uint32_t *)x1);
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
+psml_status psml_reconstruct(psml_ring ring, const void *x0, const void *x1, int64_t n, void *x,
+                             psml_stream stream) {
+    PSML_TRY(check_ring(ring));
+    if (n < 0) return fail(PSML_ERR_SHAPE, "n < 0");
+    if (n == 0) return PSML_OK;
+    PSML_TRY(check_ptrs({x0, x1, x}));
+    cudaStream_t s = (cudaStream_t)stream;
+    if (ring.l == 64) add_kernel<uint64_t><<<grid_for(n, 256), 256, 0, s>>>((const uint64_t *)x0, (const uint64_t *)x1, n, (uint64_t *)x);
+    else add_kernel<uint32_t><<<grid_for(n, 256), 256, 0, s>>>((const uint32_t *)x0, (const uint32_t *)x1, n, (uint32_t *)x);
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
+// ------------------------------------------------------------------------------------------------
+// dealer
+// ------------------------------------------------------------------------------------------------
+template <typename T>
+static psml_status triplet_gen_t(Ctx *c, uint64_t seed, uint64_t cid, int64_t M, int64_t K, int64_t N,
+                                 void *const U[2], void *const V[2], void *const Z[2], cudaStream_t s) {
+    // workspace: U sum (MK) + V sum (KN) + split-K partial (MN)
+    const int64_t words = M * K + K * N + M * N;
+    PSML_TRY(c->ensure_ws(sizeof(T) * words));
+    T *Us = (T *)c->ws, *Vs = Us + M * K, *part = Vs + K * N;
+    dealer_pair_kernel<T><<<grid_for(M * K / 8 + 1, 256), 256, 0, s>>>(make_key(seed, TAG_U0, cid), make_key(seed, TAG_U1, cid), M * K,
+                                                                       (T *)U[0], (T *)U[1], Us);
+    PSML_LAUNCH_CHECK();
+    dealer_pair_kernel<T><<<grid_for(K * N / 8 + 1, 256), 256, 0, s>>>(make_key(seed, TAG_V0, cid), make_key(seed, TAG_V1, cid), K * N,
+                                                                       (T *)V[0], (T *)V[1], Vs);
+    PSML_LAUNCH_CHECK();
+    // Z = (U0+U1)(V0+V1): through the plain ring GEMM (tcgen05 when it pays), then the split
+    if (c->use_tc(M, K, N)) {
+        size_t need = tc_ring_gemm_ws_bytes(8 * (int)sizeof(T), M, K, N);
+        // plain GEMM into Z[1], then Z0 = PRG, Z1 -= Z0 (fused tiny kernel)
+        PSML_TRY(c->ensure_ws(sizeof(T) * words + need));
+        Us = (T *)c->ws; Vs = Us + M * K;
+        psml_status st = tc_ring_gemm_plain(8 * (int)sizeof(T), Us, Vs, M, K, N, Z[1],
+                                            (char *)c->ws + sizeof(T) * words, need, s);
+        if (st == PSML_OK) {
+            prg_kernel<T, 1><<<grid_for(M * N / 8 + 2, 256), 256, 0, s>>>(make_key(seed, TAG_Z0, cid), 0, M * N, (T *)Z[0],
+                                                                          (const T *)Z[1], (T *)Z[1]);
+            PSML_LAUNCH_CHECK();
+            return PSML_OK;
+        }
+        if (st != PSML_ERR_UNSUPPORTED) return st;
+    }
+    DealerOps<T> ops;
+    ops.U0 = (const T *)U[0]; ops.U1 = (const T *)U[1]; ops.V0 = (const T *)V[0]; ops.V1 = (const T *)V[1];
+    ops.Z0 = (T *)Z[0]; ops.Z1 = (T *)Z[1];
+    ops.kz0 = make_key(seed, TAG_Z0, cid);
+    ops.M = M; ops.N = N; ops.Kext = K;
+    return launch_ring_gemm<T, DealerOps<T>>(ops, part, M * N, s, c->sm_count);
+}
+
+psml_status psml_triplet_gen(psml_ctx ctx, uint64_t seed, uint64_t call_id, int64_t M, int64_t K, int64_t N,
+                             void *const U[2], void *const V[2], void *const Z[2], psml_stream stream) {
+    if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
+    Ctx *c = reinterpret_cast<Ctx *>(ctx);
+    if (M <= 0 || K <= 0 || N <= 0) return fail(PSML_ERR_SHAPE, "M, K, N must be positive");
+    if (!U || !V || !Z) return fail(PSML_ERR_INVALID, "null pair array");
+    PSML_TRY(check_ptrs({U[0], U[1], V[0], V[1], Z[0], Z[1]}));
+    cudaStream_t s = (cudaStream_t)stream;
+    if (c->ring.l == 64) return triplet_gen_t<uint64_t>(c, seed, call_id, M, K, N, U, V, Z, s);
+    return triplet_gen_t<uint32_t>(c, seed, call_id, M, K, N, U, V, Z, s);
+}
+
+psml_status psml_hadamard_triplet_gen(psml_ring ring, uint64_t seed, uint64_t call_id, int64_t n, void *const U[2],
+                                      void *const V[2], void *const Z[2], psml_stream stream) {
+    PSML_TRY(check_ring(ring));
+    if (n < 0) return fail(PSML_ERR_SHAPE, "n < 0");
+    if (n == 0) return PSML_OK;
+    if (!U || !V || !Z) return fail(PSML_ERR_INVALID, "null pair array");
+    PSML_TRY(check_ptrs({U[0], U[1], V[0], V[1], Z[0], Z[1]}));
+    cudaStream_t s = (cudaStream_t)stream;
+    if (ring.l == 64)
+        return hadamard_triplet_launch<uint64_t>(seed, call_id, n, U, V, Z, s);
+    return hadamard_triplet_launch<uint32_t>(seed, call_id, n, U, V, Z, s);
+}
+
+int64_t psml_msb_material_words(psml_ring ring, int64_t n) {
+    if (ring.l != 32 && ring.l != 64) return -1;
+    return (int64_t)(6 * ilog2_int(ring.l) + 2) * n;
+}
+
+psml_status psml_msb_dealer(psml_ring ring, uint64_t seed, uint64_t call_id, int64_t n, void *const mat[2],
+                            psml_stream stream) {
+    PSML_TRY(check_ring(ring));
+    if (n < 0) return fail(PSML_ERR_SHAPE, "n < 0");
+    if (n == 0) return PSML_OK;
+    if (!mat) return fail(PSML_ERR_INVALID, "null pair array");
+    PSML_TRY(check_ptrs({mat[0], mat[1]}));
+    cudaStream_t s = (cudaStream_t)stream;
+    if (ring.l == 64) return msb_dealer_launch<uint64_t>(seed, call_id, n, mat, s);
+    return msb_dealer_launch<uint32_t>(seed, call_id, n, mat, s);
+}
+
+// ------------------------------------------------------------------------------------------------
+// server side
+// ------------------------------------------------------------------------------------------------
+template <typename T>
+static psml_status secure_matmul_t(Ctx *c, const void *const A[2], const void *const B[2], const void *const U[2],
+                                   const void *const V[2], const void *const Z[2], int64_t M, int64_t K, int64_t N,
+                                   int32_t flags, int32_t trunc, void *const C[2], const psml_trace *tr,
+                                   cudaStream_t s) {
+    const T *a[2] = {(const T *)A[0], (const T *)A[1]}, *b[2] = {(const T *)B[0], (const T *)B[1]};
+    const T *u[2] = {(const T *)U[0], (const T *)U[1]}, *v[2] = {(const T *)V[0], (const T *)V[1]};
+    const T *z[2] = {(const T *)Z[0], (const T *)Z[1]};
+    T *cc[2] = {(T *)C[0], (T *)C[1]};
+    if (!tr && !(flags & PSML_PAPER_FORM) && c->use_tc(M, 2 * K, N)) {
+        psml_status st = tc_beaver_matmul<T>(c, a, b, u, v, z, M, K, N, flags, trunc, cc, s);
+        if (st != PSML_ERR_UNSUPPORTED) return st;
+    }
+    const int64_t words = beaver_ws_words<T>(M, K, N);
+    PSML_TRY(c->ensure_ws(sizeof(T) * words));
+    T *ws = (T *)c->ws;
+    T *tE[2] = {tr ? (T *)tr->E[0] : nullptr, tr ? (T *)tr->E[1] : nullptr};
+    T *tF[2] = {tr ? (T *)tr->F[0] : nullptr, tr ? (T *)tr->F[1] : nullptr};
+    PSML_TRY(beaver_matmul<T>(a, b, u, v, z, M, K, N, flags, trunc, cc, ws, words, s, c->sm_count, tE, tF));
+    if (tr) PSML_TRY(trace_opened<T>(c, M, K, N, tr, s));
+    return PSML_OK;
+}
+
+psml_status psml_secure_matmul(psml_ctx ctx, const void *const A[2], const void *const B[2], const void *const U[2],
+                               const void *const V[2], const void *const Z[2], int64_t M, int64_t K, int64_t N,
+                               int32_t flags, int32_t trunc_bits, void *const C[2], const psml_trace *trace,
+                               psml_stream stream) {
+    if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
+    Ctx *c = reinterpret_cast<Ctx *>(ctx);
+    if (M <= 0 || K <= 0 || N <= 0) return fail(PSML_ERR_SHAPE, "M, K, N must be positive");
+    if (trunc_bits < 0 || trunc_bits >= c->ring.l) return fail(PSML_ERR_SHAPE, "trunc_bits must be in [0, l)");
+    if (flags & ~(PSML_TRANS_A | PSML_TRANS_B | PSML_PAPER_FORM)) return fail(PSML_ERR_INVALID, "unknown flag bits");
+    if (!A || !B || !U || !V || !Z || !C) return fail(PSML_ERR_INVALID, "null pair array");
+    PSML_TRY(check_ptrs({A[0], A[1], B[0], B[1], U[0], U[1], V[0], V[1], Z[0], Z[1], C[0], C[1]}));
+    cudaStream_t s = (cudaStream_t)stream;
+    if (c->ring.l == 64) return secure_matmul_t<uint64_t>(c, A, B, U, V, Z, M, K, N, flags, trunc_bits, C, trace, s);
+    return secure_matmul_t<uint32_t>(c, A, B, U, V, Z, M, K, N, flags, trunc_bits, C, trace, s);
+}
+
+psml_status psml_secure_hadamard(psml_ctx ctx, const void *const A[2], const void *const B[2], const void *const U[2],
+                                 const void *const V[2], const void *const Z[2], int64_t n, int32_t trunc_bits,
+                                 void *const C[2], psml_stream stream) {
+    if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
+    Ctx *c = reinterpret_cast<Ctx *>(ctx);
+    if (n < 0) return fail(PSML_ERR_SHAPE, "n < 0");
+    if (trunc_bits < 0 || trunc_bits >= c->ring.l) return fail(PSML_ERR_SHAPE, "trunc_bits must be in [0, l)");
+    if (n == 0) return PSML_OK;
+    if (!A || !B || !U || !V || !Z || !C) return fail(PSML_ERR_INVALID, "null pair array");
+    PSML_TRY(check_ptrs({A[0], A[1], B[0], B[1], U[0], U[1], V[0], V[1], Z[0], Z[1], C[0], C[1]}));
+    cudaStream_t s = (cudaStream_t)stream;
+    if (c->ring.l == 64) {
+        PSML_TRY(c->ensure_ws(sizeof(uint64_t) * 4 * n));
+        return beaver_hadamard<uint64_t>((const uint64_t *const *)A, (const uint64_t *const *)B, (const uint64_t *const *)U,
+                                         (const uint64_t *const *)V, (const uint64_t *const *)Z, n, trunc_bits,
+                                         (uint64_t *const *)C, (uint64_t *)c->ws, s);
+    }
+    PSML_TRY(c->ensure_ws(sizeof(uint32_t) * 4 * n));
+    return beaver_hadamard<uint32_t>((const uint32_t *const *)A, (const uint32_t *const *)B, (const uint32_t *const *)U,
+                                     (const uint32_t *const *)V, (const uint32_t *const *)Z, n, trunc_bits,
+                                     (uint32_t *const *)C, (uint32_t *)c->ws, s);
+}
+
+psml_status psml_truncate(psml_ring ring, int32_t party, void *x_i, int64_t n, int32_t bits, psml_stream stream) {
+    PSML_TRY(check_ring(ring));
+    if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
+    if (n < 0 || bits < 0 || bits >= ring.l) return fail(PSML_ERR_SHAPE, "bad n or bits");
+    if (n == 0 || bits == 0) return PSML_OK;
+    PSML_TRY(check_ptrs({x_i}));
+    cudaStream_t s = (cudaStream_t)stream;
+    if (ring.l == 64) truncate_kernel<uint64_t><<<grid_for(n, 256), 256, 0, s>>>((uint64_t *)x_i, n, party, bits);
+    else truncate_kernel<uint32_t><<<grid_for(n, 256), 256, 0, s>>>((uint32_t *)x_i, n, party, bits);
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
+template <typename T>
+static psml_status activation_t(Ctx *c, int what, const void *const x[2], int64_t n, const void *const mat[2],
+                                void *const msbA[2], void *const msbB[2], const void *const U[2],
+                                const void *const V[2], const void *const Z[2], void *const y[2],
+                                void *const drelu[2], cudaStream_t s) {
+    const int64_t nn = what == 2 ? 2 * n : n;  // Eq. 9 runs the chain on [x + 1/2 ; x - 1/2]
+    PSML_TRY(c->ensure_ws(sizeof(T) * msb_ws_words<T>(nn)));
+    const T half = (T)1 << (c->ring.frac_bits > 0 ? c->ring.frac_bits - 1 : 0);
+    return msb_chain<T>((const T *const *)x, nn, (const T *const *)mat, what == 2 ? 1 : 0, half, what,
+                        (T *const *)msbA, (T *const *)msbB, (T *const *)drelu, (const T *const *)U,
+                        (const T *const *)V, (const T *const *)Z, (T *const *)y, nullptr, nullptr, (T *)c->ws, s);
+}
+
+psml_status psml_secure_msb(psml_ctx ctx, const void *const x[2], int64_t n, const void *const mat[2],
+                            void *const msbA[2], void *const msbB[2], psml_stream stream) {
+    if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
+    Ctx *c = reinterpret_cast<Ctx *>(ctx);
+    if (n < 0) return fail(PSML_ERR_SHAPE, "n < 0");
+    if (n == 0) return PSML_OK;
+    if (!x || !mat || !msbA) return fail(PSML_ERR_INVALID, "null pair array");
+    PSML_TRY(check_ptrs({x[0], x[1], mat[0], mat[1], msbA[0], msbA[1]}));
+    cudaStream_t s = (cudaStream_t)stream;
+    if (c->ring.l == 64) return activation_t<uint64_t>(c, 0, x, n, mat, msbA, msbB, nullptr, nullptr, nullptr, nullptr, nullptr, s);
+    return activation_t<uint32_t>(c, 0, x, n, mat, msbA, msbB, nullptr, nullptr, nullptr, nullptr, nullptr, s);
+}
+
+psml_status psml_secure_relu(psml_ctx ctx, const void *const x[2], int64_t n, const void *const mat[2],
+                             const void *const U[2], const void *const V[2], const void *const Z[2], void *const y[2],
+                             void *const drelu[2], psml_stream stream) {
+    if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
+    Ctx *c = reinterpret_cast<Ctx *>(ctx);
+    if (n < 0) return fail(PSML_ERR_SHAPE, "n < 0");
+    if (n == 0) return PSML_OK;
+    if (!x || !mat || !U || !V || !Z || !y) return fail(PSML_ERR_INVALID, "null pair array");
+    PSML_TRY(check_ptrs({x[0], x[1], mat[0], mat[1], U[0], U[1], V[0], V[1], Z[0], Z[1], y[0], y[1]}));
+    cudaStream_t s = (cudaStream_t)stream;
+    if (c->ring.l == 64) return activation_t<uint64_t>(c, 1, x, n, mat, nullptr, nullptr, U, V, Z, y, drelu, s);
+    return activation_t<uint32_t>(c, 1, x, n, mat, nullptr, nullptr, U, V, Z, y, drelu, s);
+}
+
+psml_status psml_secure_eq9(psml_ctx ctx, const void *const x[2], int64_t n, const void *const mat[2],
+                            const void *const U[2], const void *const V[2], const void *const Z[2], void *const y[2],
+                            psml_stream stream) {
+    if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
+    Ctx *c = reinterpret_cast<Ctx *>(ctx);
+    if (n < 0) return fail(PSML_ERR_SHAPE, "n < 0");
+    if (n == 0) return PSML_OK;
+    if (!x || !mat || !U || !V || !Z || !y) return fail(PSML_ERR_INVALID, "null pair array");
+    PSML_TRY(check_ptrs({x[0], x[1], mat[0], mat[1], U[0], U[1], V[0], V[1], Z[0], Z[1], y[0], y[1]}));
+    cudaStream_t s = (cudaStream_t)stream;
+    if (c->ring.l == 64) return activation_t<uint64_t>(c, 2, x, n, mat, nullptr, nullptr, U, V, Z, y, nullptr, s);
+    return activation_t<uint32_t>(c, 2, x, n, mat, nullptr, nullptr, U, V, Z, y, nullptr, s);
+}
+
+template <typename T>
+static psml_status ring_gemm_t(Ctx *c, const void *A, const void *B, int64_t M, int64_t K, int64_t N, void *C,
+                               cudaStream_t s) {
+    if (c->use_tc(M, K, N)) {
+        size_t need = tc_ring_gemm_ws_bytes(8 * (int)sizeof(T), M, K, N);
+        PSML_TRY(c->ensure_ws(need));
+        psml_status st = tc_ring_gemm_plain(8 * (int)sizeof(T), A, B, M, K, N, C, c->ws, c->ws_bytes, s);
+        if (st != PSML_ERR_UNSUPPORTED) return st;
+    }
+    PSML_TRY(c->ensure_ws(sizeof(T) * M * N));
+    PlainOps<T> ops;
+    ops.A = (const T *)A; ops.B = (const T *)B; ops.C = (T *)C;
+    ops.M = M; ops.N = N; ops.Kext = K;
+    return launch_ring_gemm<T, PlainOps<T>>(ops, (T *)c->ws, M * N, s, c->sm_count);
+}
+
+psml_status psml_ring_gemm(psml_ctx ctx, const void *A, const void *B, int64_t M, int64_t K, int64_t N, void *C,
+                           psml_stream stream) {
+    if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
+    Ctx *c = reinterpret_cast<Ctx *>(ctx);
+    if (M <= 0 || K <= 0 || N <= 0) return fail(PSML_ERR_SHAPE, "M, K, N must be positive");
+    PSML_TRY(check_ptrs({A, B, C}));
+    cudaStream_t s = (cudaStream_t)stream;
+    if (c->ring.l == 64) return ring_gemm_t<uint64_t>(c, A, B, M, K, N, C, s);
+    return ring_gemm_t<uint32_t>(c, A, B, M, K, N, C, s);
+}
+

@@ -1,0 +1,76 @@
+// engine.h -- internal declarations shared by engine.cu, model.cu and gemm_tc.cu.
+#pragma once
+#include <algorithm>
+#include <initializer_list>
+
+#include "ops.cuh"
+
+namespace psml {
+
+psml_status check_ring(psml_ring r);
+psml_status check_ptrs(std::initializer_list<const void *> ps);
+int current_sm_count();
+
+struct Ctx {
+    psml_ring ring{64, 13};
+    int backend = 0;    // 0 auto, 1 CUDA-core, 2 tcgen05
+    int sm_count = 148;
+    bool tc_ok = false;
+    void *ws = nullptr;
+    size_t ws_bytes = 0;
+    psml_status ensure_ws(size_t bytes);
+    // tcgen05 limb GEMM pays once the product has enough tiles and depth (gemm_tc.cu).
+    bool use_tc(int64_t M, int64_t Kext, int64_t N) const {
+        if (!tc_ok || backend == 1) return false;
+        if (backend == 2) return true;
+        return M >= 256 && N >= 128 && Kext >= 256 && M * N >= (int64_t)1 << 18;
+    }
+};
+
+// ------------------------------------------------------------------------------------------------
+// launch helpers (templates, used by engine.cu and model.cu)
+// ------------------------------------------------------------------------------------------------
+template <typename T>
+psml_status hadamard_triplet_launch(uint64_t seed, uint64_t cid, int64_t n, void *const U[2], void *const V[2],
+                                    void *const Z[2], cudaStream_t s) {
+    Pair<T> u{{(T *)U[0], (T *)U[1]}}, v{{(T *)V[0], (T *)V[1]}}, z{{(T *)Z[0], (T *)Z[1]}};
+    const int64_t nblk = (n + PerBlock<T>::value - 1) / PerBlock<T>::value;
+    hadamard_triplet_kernel<T><<<grid_for(nblk, 128, 148 * 32), 128, 0, s>>>(
+        make_key(seed, TAG_U0, cid), make_key(seed, TAG_U1, cid), make_key(seed, TAG_V0, cid),
+        make_key(seed, TAG_V1, cid), make_key(seed, TAG_Z0, cid), n, u, v, z);
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
+template <typename T>
+psml_status msb_dealer_launch(uint64_t seed, uint64_t cid, int64_t n, void *const mat[2], cudaStream_t s) {
+    const int L = ilog2_int(8 * (int)sizeof(T));
+    const int64_t nblk = (n + PerBlock<T>::value - 1) / PerBlock<T>::value;
+    dim3 grid((unsigned)grid_for(nblk, 128, 148 * 8), (unsigned)(2 * L + 1));
+    msb_dealer_kernel<T><<<grid, 128, 0, s>>>(seed, cid, n, L, (T *)mat[0], (T *)mat[1]);
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
+// opened values for psml_trace: E = E_0 + E_1, F = F_0 + F_1 (from the trace's E_i/F_i copies)
+template <typename T>
+psml_status trace_opened(Ctx *c, int64_t M, int64_t K, int64_t N, const psml_trace *tr, cudaStream_t s) {
+    (void)c;
+    if (tr->E_open && tr->E[0] && tr->E[1]) {
+        add_kernel<T><<<grid_for(M * K, 256), 256, 0, s>>>((const T *)tr->E[0], (const T *)tr->E[1], M * K, (T *)tr->E_open);
+        PSML_LAUNCH_CHECK();
+    }
+    if (tr->F_open && tr->F[0] && tr->F[1]) {
+        add_kernel<T><<<grid_for(K * N, 256), 256, 0, s>>>((const T *)tr->F[0], (const T *)tr->F[1], K * N, (T *)tr->F_open);
+        PSML_LAUNCH_CHECK();
+    }
+    return PSML_OK;
+}
+
+// tcgen05 Beaver product (gemm_tc.cu); PSML_ERR_UNSUPPORTED = take the CUDA-core path.
+template <typename T>
+psml_status tc_beaver_matmul(Ctx *c, const T *const A[2], const T *const B[2], const T *const U[2],
+                             const T *const V[2], const T *const Z[2], int64_t M, int64_t K, int64_t N, int flags,
+                             int trunc, T *const C[2], cudaStream_t s);
+
+}  // namespace psml

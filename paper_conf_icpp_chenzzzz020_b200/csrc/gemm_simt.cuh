@@ -1,0 +1,400 @@
+// gemm_simt.cuh -- CUDA-core ring GEMM in Z_{2^l} (l = 64: uint64 IMAD.WIDE chains; l = 32:
+// uint32 IMAD) with pluggable operand loaders and epilogues.
+//
+// The loaders fuse the Beaver opening and the Eq. 8 K-concatenation of PAPER.md L175:
+//   party i computes C_i = [i.E + U_i | E] . [F ; V_i] + Z_i with E = E_0 + E_1, F = F_0 + F_1
+// read straight from both parties' masked messages, so D' = i.E + U_i is never materialised.
+// Two kernels:
+//   ring_gemm_tiled  BM x BN tiles, register-blocked TM x TN per thread, double-buffered smem
+//   ring_gemv        one warp per output row for N <= 16 (w^T x shapes of BASELINE configs 1-2,
+//                    the MLP output layer, the CNN conv im2col GEMM with N = C_out = 16)
+// Both support split-K with exact uint64/uint32 atomics (ring addition is associative and
+// exact), finished by ring_gemm_finalize which applies the epilogue.
+#pragma once
+#include <algorithm>
+
+#include "common.cuh"
+
+namespace psml {
+
+// ---------------------------------------------------------------------------------------------
+// operand/epilogue policies.  Each provides:
+//   nparty, M, N, Kext; T a(p, m, k); T b(p, k, n); void store(p, m, n, T acc)
+// ---------------------------------------------------------------------------------------------
+template <typename T>
+struct PlainOps {
+    const T *A, *B;
+    T *C;
+    int64_t M, N, Kext;
+    static constexpr int nparty = 1;
+    __device__ __forceinline__ T a(int, int64_t m, int64_t k) const { return A[m * Kext + k]; }
+    __device__ __forceinline__ T b(int, int64_t k, int64_t n) const { return B[k * N + n]; }
+    __device__ __forceinline__ void store(int, int64_t m, int64_t n, T acc) const { C[m * N + n] = acc; }
+};
+
+// Dealer: Z = (U_0 + U_1)(V_0 + V_1); Z_0 = PRG("Z0"), Z_1 = Z - Z_0 (Eqs. 2-3, R4).
+template <typename T>
+struct DealerOps {
+    const T *U0, *U1, *V0, *V1;
+    T *Z0, *Z1;
+    PrgKey kz0;
+    int64_t M, N, Kext;
+    static constexpr int nparty = 1;
+    __device__ __forceinline__ T a(int, int64_t m, int64_t k) const {
+        return U0[m * Kext + k] + U1[m * Kext + k];
+    }
+    __device__ __forceinline__ T b(int, int64_t k, int64_t n) const {
+        return V0[k * N + n] + V1[k * N + n];
+    }
+    __device__ __forceinline__ void store(int, int64_t m, int64_t n, T acc) const {
+        T z0 = prg_elem<T>(kz0, (uint64_t)(m * N + n));
+        Z0[m * N + n] = z0;
+        Z1[m * N + n] = acc - z0;
+    }
+};
+
+// Beaver product, both parties, Eq. 8 shape.  E/F are opened on the fly from the two parties'
+// messages mE[0], mE[1] (M x K) and mF[0], mF[1] (K x N).  form 0 (BJ canonical):
+//   [i.E + U_i | E] . [F ; V_i];  form 1 (Eq. 6/8): [A_i - i.E | E] . [F ; B_i].
+template <typename T>
+struct BeaverOps {
+    const T *mE0, *mE1, *mF0, *mF1;
+    const T *U[2], *V[2], *Z[2];
+    const T *A[2], *B[2];   // only for form 1 (op(A) / op(B) layouts, see transA/transB)
+    T *C[2];
+    int64_t M, N, K, Kext;  // Kext = 2K
+    int form, transA, transB, trunc;
+    static constexpr int nparty = 2;
+    __device__ __forceinline__ T opA(int p, int64_t m, int64_t k) const {
+        return transA ? A[p][k * M + m] : A[p][m * K + k];
+    }
+    __device__ __forceinline__ T opB(int p, int64_t k, int64_t n) const {
+        return transB ? B[p][n * K + k] : B[p][k * N + n];
+    }
+    __device__ __forceinline__ T a(int p, int64_t m, int64_t k) const {
+        if (k < K) {
+            T e = mE0[m * K + k] + mE1[m * K + k];
+            return form == 0 ? (T)((T)p * e + U[p][m * K + k]) : (T)(opA(p, m, k) - (T)p * e);
+        }
+        k -= K;
+        return mE0[m * K + k] + mE1[m * K + k];
+    }
+    __device__ __forceinline__ T b(int p, int64_t k, int64_t n) const {
+        if (k < K) return mF0[k * N + n] + mF1[k * N + n];
+        k -= K;
+        return form == 0 ? V[p][k * N + n] : opB(p, k, n);
+    }
+    __device__ __forceinline__ void store(int p, int64_t m, int64_t n, T acc) const {
+        T c = acc + Z[p][m * N + n];
+        C[p][m * N + n] = trunc_share<T>(c, p, trunc);
+    }
+};
+
+// Convolution as im2col ring GEMM with the mask applied to the UN-EXPANDED input (R17):
+// E_X = E_0 + E_1 over B x (C H W); im2col row r = (b, oy, ox), col c = (ch, ky, kx).
+// transposed = 0: A' = im2col(.)            (rows B*OH*OW, K = C*k*k)   -- conv forward
+// transposed = 1: A' = im2col(.)^T          (rows C*k*k,  K = B*OH*OW)  -- weight gradient
+struct ConvGeom {
+    int C, H, W, k, OH, OW;
+};
+
+template <typename T>
+struct ConvBeaverOps {
+    const T *mE0, *mE1;     // masked raw input messages, B x CHW
+    const T *UX[2];         // raw-input masks per party, B x CHW
+    const T *mF0, *mF1;     // masked B-operand messages, K x N
+    const T *V[2], *Z[2];
+    T *C[2];
+    ConvGeom g;
+    int64_t M, N, K, Kext;
+    int transposed, trunc;
+    static constexpr int nparty = 2;
+    __device__ __forceinline__ int64_t src(int64_t r, int64_t c) const {
+        int64_t plane = (int64_t)g.OH * g.OW;
+        int64_t b = r / plane, rem = r - b * plane;
+        int oy = (int)(rem / g.OW), ox = (int)(rem - (int64_t)oy * g.OW);
+        int kk = g.k * g.k;
+        int ch = (int)(c / kk), r2 = (int)(c - (int64_t)ch * kk);
+        int ky = r2 / g.k, kx = r2 - ky * g.k;
+        return b * ((int64_t)g.C * g.H * g.W) + ((int64_t)ch * g.H + oy + ky) * g.W + ox + kx;
+    }
+    __device__ __forceinline__ T a(int p, int64_t m, int64_t k) const {
+        bool first = k < K;
+        if (!first) k -= K;
+        int64_t s = transposed ? src(k, m) : src(m, k);
+        T e = mE0[s] + mE1[s];
+        return first ? (T)((T)p * e + UX[p][s]) : e;
+    }
+    __device__ __forceinline__ T b(int p, int64_t k, int64_t n) const {
+        if (k < K) return mF0[k * N + n] + mF1[k * N + n];
+        k -= K;
+        return V[p][k * N + n];
+    }
+    __device__ __forceinline__ void store(int p, int64_t m, int64_t n, T acc) const {
+        T c = acc + Z[p][m * N + n];
+        C[p][m * N + n] = trunc_share<T>(c, p, trunc);
+    }
+};
+
+// Dealer for the conv triplet: Z = im2col(U_0+U_1) (.^T) . (V_0+V_1), Z_1 = Z - PRG("Z0").
+template <typename T>
+struct ConvDealerOps {
+    const T *U0, *U1, *V0, *V1;
+    T *Z0, *Z1;
+    PrgKey kz0;
+    ConvGeom g;
+    int64_t M, N, Kext;
+    int transposed;
+    static constexpr int nparty = 1;
+    __device__ __forceinline__ int64_t src(int64_t r, int64_t c) const {
+        int64_t plane = (int64_t)g.OH * g.OW;
+        int64_t b = r / plane, rem = r - b * plane;
+        int oy = (int)(rem / g.OW), ox = (int)(rem - (int64_t)oy * g.OW);
+        int kk = g.k * g.k;
+        int ch = (int)(c / kk), r2 = (int)(c - (int64_t)ch * kk);
+        int ky = r2 / g.k, kx = r2 - ky * g.k;
+        return b * ((int64_t)g.C * g.H * g.W) + ((int64_t)ch * g.H + oy + ky) * g.W + ox + kx;
+    }
+    __device__ __forceinline__ T a(int, int64_t m, int64_t k) const {
+        int64_t s = transposed ? src(k, m) : src(m, k);
+        return U0[s] + U1[s];
+    }
+    __device__ __forceinline__ T b(int, int64_t k, int64_t n) const {
+        return V0[k * N + n] + V1[k * N + n];
+    }
+    __device__ __forceinline__ void store(int, int64_t m, int64_t n, T acc) const {
+        T z0 = prg_elem<T>(kz0, (uint64_t)(m * N + n));
+        Z0[m * N + n] = z0;
+        Z1[m * N + n] = acc - z0;
+    }
+};
+
+// ---------------------------------------------------------------------------------------------
+// tiled kernel
+// ---------------------------------------------------------------------------------------------
+template <typename T, int BM, int BN, int BK, int TM, int TN, class Ops>
+__global__ void __launch_bounds__((BM / TM) * (BN / TN))
+ring_gemm_tiled(Ops ops, int64_t k_per_split, T *__restrict__ partial) {
+    constexpr int NT = (BM / TM) * (BN / TN);
+    constexpr int A_PER = (BM * BK) / NT;
+    constexpr int B_PER = (BK * BN) / NT;
+    static_assert(A_PER * NT == BM * BK && B_PER * NT == BK * BN, "tile/thread mismatch");
+    __shared__ T As[2][BK][BM];
+    __shared__ T Bs[2][BK][BN];
+
+    const int p = blockIdx.z % Ops::nparty;
+    const int split = blockIdx.z / Ops::nparty;
+    const int64_t m0 = (int64_t)blockIdx.y * BM, n0 = (int64_t)blockIdx.x * BN;
+    const int64_t kbeg = (int64_t)split * k_per_split;
+    const int64_t kend = min(ops.Kext, kbeg + k_per_split);
+    const int tid = threadIdx.x;
+    const int tx = tid % (BN / TN), ty = tid / (BN / TN);
+
+    T acc[TM][TN];
+#pragma unroll
+    for (int i = 0; i < TM; ++i)
+#pragma unroll
+        for (int j = 0; j < TN; ++j) acc[i][j] = 0;
+
+    T ra[A_PER], rb[B_PER];
+    auto load = [&](int64_t k0) {
+#pragma unroll
+        for (int t = 0; t < A_PER; ++t) {
+            int idx = tid + t * NT;
+            int mm = idx / BK, kk = idx % BK;          // coalesced along k
+            int64_t m = m0 + mm, k = k0 + kk;
+            ra[t] = (m < ops.M && k < kend) ? ops.a(p, m, k) : (T)0;
+        }
+#pragma unroll
+        for (int t = 0; t < B_PER; ++t) {
+            int idx = tid + t * NT;
+            int kk = idx / BN, nn = idx % BN;          // coalesced along n
+            int64_t k = k0 + kk, n = n0 + nn;
+            rb[t] = (n < ops.N && k < kend) ? ops.b(p, k, n) : (T)0;
+        }
+    };
+    auto stash = [&](int buf) {
+#pragma unroll
+        for (int t = 0; t < A_PER; ++t) {
+            int idx = tid + t * NT;
+            As[buf][idx % BK][idx / BK] = ra[t];
+        }
+#pragma unroll
+        for (int t = 0; t < B_PER; ++t) {
+            int idx = tid + t * NT;
+            Bs[buf][idx / BN][idx % BN] = rb[t];
+        }
+    };
+
+    int buf = 0;
+    if (kbeg < kend) {
+        load(kbeg);
+        stash(0);
+    }
+    __syncthreads();
+    for (int64_t k0 = kbeg; k0 < kend; k0 += BK) {
+        const bool more = k0 + BK < kend;
+        if (more) load(k0 + BK);
+#pragma unroll
+        for (int kk = 0; kk < BK; ++kk) {
+            T av[TM], bv[TN];
+#pragma unroll
+            for (int i = 0; i < TM; ++i) av[i] = As[buf][kk][ty + i * (BM / TM)];
+#pragma unroll
+            for (int j = 0; j < TN; ++j) bv[j] = Bs[buf][kk][tx + j * (BN / TN)];
+#pragma unroll
+            for (int i = 0; i < TM; ++i)
+#pragma unroll
+                for (int j = 0; j < TN; ++j) acc[i][j] += av[i] * bv[j];
+        }
+        if (more) {
+            stash(buf ^ 1);
+            __syncthreads();
+            buf ^= 1;
+        }
+    }
+    if (partial == nullptr) {
+#pragma unroll
+        for (int i = 0; i < TM; ++i) {
+            int64_t m = m0 + ty + i * (BM / TM);
+            if (m >= ops.M) continue;
+#pragma unroll
+            for (int j = 0; j < TN; ++j) {
+                int64_t n = n0 + tx + j * (BN / TN);
+                if (n < ops.N) ops.store(p, m, n, acc[i][j]);
+            }
+        }
+    } else {
+#pragma unroll
+        for (int i = 0; i < TM; ++i) {
+            int64_t m = m0 + ty + i * (BM / TM);
+            if (m >= ops.M) continue;
+#pragma unroll
+            for (int j = 0; j < TN; ++j) {
+                int64_t n = n0 + tx + j * (BN / TN);
+                if (n >= ops.N) continue;
+                T *dst = partial + ((int64_t)p * ops.M + m) * ops.N + n;
+                if (sizeof(T) == 8) atomicAdd((unsigned long long *)dst, (unsigned long long)acc[i][j]);
+                else atomicAdd((unsigned int *)dst, (unsigned int)acc[i][j]);
+            }
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------------------------
+// warp-per-row kernel for N <= NN (NN in {1, 2, 4, 8, 16})
+// ---------------------------------------------------------------------------------------------
+template <typename T>
+__device__ __forceinline__ T warp_sum(T v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    return v;
+}
+
+template <typename T, int NN, class Ops>
+__global__ void __launch_bounds__(256) ring_gemv(Ops ops, int64_t k_per_split, int splits,
+                                                 T *__restrict__ partial) {
+    const int lane = threadIdx.x & 31;
+    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t rows = ops.M * Ops::nparty * splits;
+    if (gw >= rows) return;
+    const int split = (int)(gw % splits);
+    const int64_t pm = gw / splits;
+    const int p = (int)(pm % Ops::nparty);
+    const int64_t m = pm / Ops::nparty;
+    const int64_t kbeg = (int64_t)split * k_per_split;
+    const int64_t kend = min(ops.Kext, kbeg + k_per_split);
+    T acc[NN];
+#pragma unroll
+    for (int j = 0; j < NN; ++j) acc[j] = 0;
+    for (int64_t k = kbeg + lane; k < kend; k += 32) {
+        T av = ops.a(p, m, k);
+#pragma unroll
+        for (int j = 0; j < NN; ++j)
+            if (j < ops.N) acc[j] += av * ops.b(p, k, j);
+    }
+#pragma unroll
+    for (int j = 0; j < NN; ++j) {
+        if (j >= ops.N) break;
+        T s = warp_sum<T>(acc[j]);
+        if (lane == j) {
+            if (partial == nullptr) ops.store(p, m, j, s);
+            else {
+                T *dst = partial + ((int64_t)p * ops.M + m) * ops.N + j;
+                if (sizeof(T) == 8) atomicAdd((unsigned long long *)dst, (unsigned long long)s);
+                else atomicAdd((unsigned int *)dst, (unsigned int)s);
+            }
+        }
+    }
+}
+
+template <typename T, class Ops>
+__global__ void ring_gemm_finalize(Ops ops, const T *__restrict__ partial) {
+    const int64_t total = ops.M * ops.N * Ops::nparty;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        int64_t p = i / (ops.M * ops.N), r = i - p * ops.M * ops.N;
+        ops.store((int)p, r / ops.N, r % ops.N, partial[i]);
+    }
+}
+
+// ---------------------------------------------------------------------------------------------
+// host-side dispatcher: picks kernel, tile and split-K; `ws` must hold nparty*M*N words when
+// split-K is chosen (ws_words reports the need; pass ws = nullptr to query).
+// ---------------------------------------------------------------------------------------------
+template <typename T, class Ops>
+psml_status launch_ring_gemm(const Ops &ops, T *ws, int64_t ws_words, cudaStream_t stream,
+                             int sm_count = 148) {
+    const int64_t M = ops.M, N = ops.N, Kx = ops.Kext;
+    if (M <= 0 || N <= 0) return PSML_OK;
+    const int64_t outs = M * N * Ops::nparty;
+    int splits = 1;
+    if (N <= 16) {
+        const int64_t warps = M * Ops::nparty;
+        const int64_t target = (int64_t)sm_count * 32;
+        if (warps < target && Kx >= 2048) {
+            splits = (int)std::min<int64_t>((target + warps - 1) / warps, Kx / 512);
+            if (splits < 1) splits = 1;
+        }
+    } else {
+        const int64_t tiles = ((M + 63) / 64) * ((N + 63) / 64) * Ops::nparty;
+        const int64_t target = (int64_t)sm_count * 2;
+        if (tiles < target && Kx >= 1024) {
+            splits = (int)std::min<int64_t>((target + tiles - 1) / tiles, Kx / 256);
+            if (splits < 1) splits = 1;
+        }
+    }
+    if (splits > 1 && (ws == nullptr || ws_words < outs)) splits = 1;  // no workspace: no split
+    T *partial = nullptr;
+    if (splits > 1) {
+        partial = ws;
+        PSML_CUDA_TRY(cudaMemsetAsync(partial, 0, sizeof(T) * outs, stream));
+    }
+    int64_t kps = (Kx + splits - 1) / splits;
+    if (N <= 16) {
+        const int64_t warps = M * Ops::nparty * splits;
+        const int blocks = (int)((warps * 32 + 255) / 256);
+        if (N == 1) ring_gemv<T, 1, Ops><<<blocks, 256, 0, stream>>>(ops, kps, splits, partial);
+        else if (N <= 2) ring_gemv<T, 2, Ops><<<blocks, 256, 0, stream>>>(ops, kps, splits, partial);
+        else if (N <= 4) ring_gemv<T, 4, Ops><<<blocks, 256, 0, stream>>>(ops, kps, splits, partial);
+        else if (N <= 8) ring_gemv<T, 8, Ops><<<blocks, 256, 0, stream>>>(ops, kps, splits, partial);
+        else ring_gemv<T, 16, Ops><<<blocks, 256, 0, stream>>>(ops, kps, splits, partial);
+    } else {
+        kps = ((kps + 15) / 16) * 16;
+        dim3 grid((unsigned)((N + 63) / 64), (unsigned)((M + 63) / 64), (unsigned)(Ops::nparty * splits));
+        ring_gemm_tiled<T, 64, 64, 16, 4, 4, Ops><<<grid, 256, 0, stream>>>(ops, kps, partial);
+    }
+    PSML_LAUNCH_CHECK();
+    if (splits > 1) {
+        ring_gemm_finalize<T, Ops><<<grid_for(outs, 256), 256, 0, stream>>>(ops, partial);
+        PSML_LAUNCH_CHECK();
+    }
+    return PSML_OK;
+}
+
+template <class Ops>
+inline int64_t ring_gemm_ws_words(const Ops &ops) {
+    return ops.M * ops.N * Ops::nparty;
+}
+
+}  // namespace psml

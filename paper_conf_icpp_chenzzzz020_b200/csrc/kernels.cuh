@@ -1,0 +1,425 @@
+// kernels.cuh -- elementwise / protocol-round kernels of libpsml (co-resident pair engine).
+//
+// Round structure: every protocol round is ONE kernel that (1) opens the
+// previous round's messages -- reading party 0's and party 1's masked words from their send
+// buffers in HBM (Eq. 5), (2) does the local computation of both parties, and (3)
+// writes this round's masked messages.  A thread owns one element for both parties, so each
+// opened word is read once and all accesses are coalesced 8-byte (l=64) / 4-byte (l=32) words.
+#pragma once
+#include "common.cuh"
+
+namespace psml {
+
+template <typename T> struct Pair { T *p[2]; };
+template <typename T> struct CPair { const T *p[2]; };
+
+// ---------------------------------------------------------------------------------------------
+// PRG fill / encode / decode / share / reconstruct  (client side)
+// ---------------------------------------------------------------------------------------------
+// One thread per ChaCha20 block; OP = 0: out = prg; 1: out = x - prg (share: x1) and x0 = prg.
+template <typename T, int OP>
+__global__ void prg_kernel(PrgKey key, uint64_t offset, int64_t n, T *__restrict__ out,
+                           const T *__restrict__ x, T *__restrict__ out2) {
+    constexpr int PB = PerBlock<T>::value;
+    const uint64_t first_blk = offset / PB;
+    const uint64_t last_blk = (offset + (uint64_t)n - 1) / PB;
+    for (uint64_t b = first_blk + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; b <= last_blk;
+         b += (uint64_t)gridDim.x * blockDim.x) {
+        uint32_t w[16];
+        chacha20_block(key, (uint32_t)b, w);
+#pragma unroll
+        for (int j = 0; j < PB; ++j) {
+            uint64_t e = b * PB + j;
+            if (e < offset || e >= offset + (uint64_t)n) continue;
+            T v = sizeof(T) == 8 ? (T)(((uint64_t)w[2 * j + 1] << 32) | w[2 * j]) : (T)w[j];
+            int64_t i = (int64_t)(e - offset);
+            if (OP == 0) out[i] = v;
+            else { out[i] = v; out2[i] = x[i] - v; }
+        }
+    }
+}
+
+template <typename T>
+__global__ void encode_kernel(const double *__restrict__ x, int64_t n, int f, T *__restrict__ v) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        long long r = __double2ll_rn(ldexp(x[i], f));   // round half to even (R3)
+        v[i] = (T)(unsigned long long)r;
+    }
+}
+
+template <typename T>
+__global__ void decode_kernel(const T *__restrict__ v, int64_t n, int f, double *__restrict__ x) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        double s = sizeof(T) == 8 ? (double)(long long)(uint64_t)v[i] : (double)(int)(uint32_t)v[i];
+        x[i] = ldexp(s, -f);
+    }
+}
+
+template <typename T>
+__global__ void add_kernel(const T *__restrict__ a, const T *__restrict__ b, int64_t n, T *__restrict__ c) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        c[i] = a[i] + b[i];
+}
+
+template <typename T>
+__global__ void truncate_kernel(T *__restrict__ x, int64_t n, int party, int d) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        x[i] = trunc_share<T>(x[i], party, d);
+}
+
+// ---------------------------------------------------------------------------------------------
+// dealer kernels (offline; Eqs. 2-3, Fig. 4; R4, R9)
+// ---------------------------------------------------------------------------------------------
+// U0,U1 (or V0,V1) streams + their sum (written to `sum`, used as the GEMM operand for Z).
+template <typename T>
+__global__ void dealer_pair_kernel(PrgKey k0, PrgKey k1, int64_t n, T *__restrict__ o0,
+                                   T *__restrict__ o1, T *__restrict__ sum) {
+    constexpr int PB = PerBlock<T>::value;
+    const int64_t nblk = (n + PB - 1) / PB;
+    for (int64_t b = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; b < nblk; b += (int64_t)gridDim.x * blockDim.x) {
+        uint32_t w0[16], w1[16];
+        chacha20_block(k0, (uint32_t)b, w0);
+        chacha20_block(k1, (uint32_t)b, w1);
+#pragma unroll
+        for (int j = 0; j < PB; ++j) {
+            int64_t e = b * PB + j;
+            if (e >= n) break;
+            T v0 = sizeof(T) == 8 ? (T)(((uint64_t)w0[2 * j + 1] << 32) | w0[2 * j]) : (T)w0[j];
+            T v1 = sizeof(T) == 8 ? (T)(((uint64_t)w1[2 * j + 1] << 32) | w1[2 * j]) : (T)w1[j];
+            o0[e] = v0; o1[e] = v1;
+            if (sum) sum[e] = v0 + v1;
+        }
+    }
+}
+
+template <typename T>
+__device__ __forceinline__ T word_of(const uint32_t *w, int j) {
+    return sizeof(T) == 8 ? (T)(((uint64_t)w[2 * j + 1] << 32) | w[2 * j]) : (T)w[j];
+}
+
+// Hadamard triplet: Z_1 = (U0+U1)(V0+V1) - Z0, elementwise.
+template <typename T>
+__global__ void hadamard_triplet_kernel(PrgKey ku0, PrgKey ku1, PrgKey kv0, PrgKey kv1, PrgKey kz0,
+                                        int64_t n, Pair<T> U, Pair<T> V, Pair<T> Z) {
+    constexpr int PB = PerBlock<T>::value;
+    const int64_t nblk = (n + PB - 1) / PB;
+    for (int64_t b = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; b < nblk; b += (int64_t)gridDim.x * blockDim.x) {
+        uint32_t a0[16], a1[16], c0[16], c1[16], z[16];
+        chacha20_block(ku0, (uint32_t)b, a0);
+        chacha20_block(ku1, (uint32_t)b, a1);
+        chacha20_block(kv0, (uint32_t)b, c0);
+        chacha20_block(kv1, (uint32_t)b, c1);
+        chacha20_block(kz0, (uint32_t)b, z);
+#pragma unroll
+        for (int j = 0; j < PB; ++j) {
+            int64_t e = b * PB + j;
+            if (e >= n) break;
+            T u0 = word_of<T>(a0, j), u1 = word_of<T>(a1, j), v0 = word_of<T>(c0, j), v1 = word_of<T>(c1, j);
+            T z0 = word_of<T>(z, j);
+            U.p[0][e] = u0; U.p[1][e] = u1; V.p[0][e] = v0; V.p[1][e] = v1;
+            Z.p[0][e] = z0; Z.p[1][e] = (T)((u0 + u1) * (v0 + v1)) - z0;
+        }
+    }
+}
+
+// MSB material: blockIdx.y = AND index t (0 .. 2L-1) or 2L for the daBit.
+template <typename T>
+__global__ void msb_dealer_kernel(uint64_t seed, uint64_t call_id, int64_t n, int L, T *__restrict__ m0,
+                                  T *__restrict__ m1) {
+    constexpr int PB = PerBlock<T>::value;
+    const int t = blockIdx.y;
+    const int64_t nblk = (n + PB - 1) / PB;
+    for (int64_t b = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; b < nblk; b += (int64_t)gridDim.x * blockDim.x) {
+        if (t < 2 * L) {
+            uint32_t wa0[16], wa1[16], wb0[16], wb1[16], wc0[16];
+            chacha20_block(make_key(seed, tag4('a', '0', t), call_id), (uint32_t)b, wa0);
+            chacha20_block(make_key(seed, tag4('a', '1', t), call_id), (uint32_t)b, wa1);
+            chacha20_block(make_key(seed, tag4('b', '0', t), call_id), (uint32_t)b, wb0);
+            chacha20_block(make_key(seed, tag4('b', '1', t), call_id), (uint32_t)b, wb1);
+            chacha20_block(make_key(seed, tag4('c', '0', t), call_id), (uint32_t)b, wc0);
+            T *base0 = m0 + (int64_t)t * 3 * n, *base1 = m1 + (int64_t)t * 3 * n;
+#pragma unroll
+            for (int j = 0; j < PB; ++j) {
+                int64_t e = b * PB + j;
+                if (e >= n) break;
+                T a0 = word_of<T>(wa0, j), a1 = word_of<T>(wa1, j), b0 = word_of<T>(wb0, j);
+                T b1 = word_of<T>(wb1, j), c0 = word_of<T>(wc0, j);
+                base0[e] = a0; base0[n + e] = b0; base0[2 * n + e] = c0;
+                base1[e] = a1; base1[n + e] = b1; base1[2 * n + e] = ((a0 ^ a1) & (b0 ^ b1)) ^ c0;
+            }
+        } else {
+            uint32_t w0[16], w1[16], wa[16];
+            chacha20_block(make_key(seed, TAG_R0, call_id), (uint32_t)b, w0);
+            chacha20_block(make_key(seed, TAG_R1, call_id), (uint32_t)b, w1);
+            chacha20_block(make_key(seed, TAG_RA, call_id), (uint32_t)b, wa);
+            const int64_t off = (int64_t)2 * L * 3 * n;
+#pragma unroll
+            for (int j = 0; j < PB; ++j) {
+                int64_t e = b * PB + j;
+                if (e >= n) break;
+                T r0 = word_of<T>(w0, j) & 1, r1 = word_of<T>(w1, j) & 1, ra0 = word_of<T>(wa, j);
+                m0[off + e] = r0; m1[off + e] = r1;
+                m0[off + n + e] = ra0; m1[off + n + e] = (T)(r0 ^ r1) - ra0;
+            }
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------------------------
+// Beaver masking (Eq. 4): up to 4 jobs (E_0, E_1, F_0, F_1), each dst = op(src) - mask, with an
+// optional transpose of src staged through a 32x33 shared tile.
+// ---------------------------------------------------------------------------------------------
+template <typename T>
+struct MaskJob {
+    const T *src;   // rows x cols in op layout (or cols x rows if trans)
+    const T *mask;  // rows x cols
+    T *dst;         // rows x cols
+    int64_t rows, cols;
+    int trans;
+};
+template <typename T> struct MaskJobs { MaskJob<T> j[4]; int count; };
+
+template <typename T>
+__global__ void mask_kernel(MaskJobs<T> jobs) {
+    __shared__ T tile[32][33];
+    const MaskJob<T> J = jobs.j[blockIdx.z];
+    const int64_t tiles_c = (J.cols + 31) / 32;
+    const int64_t tiles = ((J.rows + 31) / 32) * tiles_c;
+    for (int64_t t = blockIdx.x; t < tiles; t += gridDim.x) {
+        const int64_t r0 = (t / tiles_c) * 32, c0 = (t % tiles_c) * 32;
+        if (J.trans) {
+            // src stored cols x rows: read coalesced along rows, write coalesced along cols
+            __syncthreads();
+            for (int i = threadIdx.y; i < 32; i += blockDim.y) {
+                int64_t sc = c0 + i, sr = r0 + threadIdx.x;
+                tile[i][threadIdx.x] = (sc < J.cols && sr < J.rows) ? J.src[sc * J.rows + sr] : (T)0;
+            }
+            __syncthreads();
+            for (int i = threadIdx.y; i < 32; i += blockDim.y) {
+                int64_t r = r0 + i, c = c0 + threadIdx.x;
+                if (r < J.rows && c < J.cols) J.dst[r * J.cols + c] = tile[threadIdx.x][i] - J.mask[r * J.cols + c];
+            }
+        } else {
+            for (int i = threadIdx.y; i < 32; i += blockDim.y) {
+                int64_t r = r0 + i, c = c0 + threadIdx.x;
+                if (r < J.rows && c < J.cols) {
+                    int64_t o = r * J.cols + c;
+                    J.dst[o] = J.src[o] - J.mask[o];
+                }
+            }
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------------------------
+// Beaver Hadamard: round 1 masks, round 2 opens and combines (BJ form), optional truncation.
+// ---------------------------------------------------------------------------------------------
+template <typename T>
+__global__ void hadamard_mask_kernel(CPair<T> A, CPair<T> B, CPair<T> U, CPair<T> V, int64_t n,
+                                     Pair<T> mE, Pair<T> mF) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+#pragma unroll
+        for (int p = 0; p < 2; ++p) {
+            mE.p[p][i] = A.p[p][i] - U.p[p][i];
+            mF.p[p][i] = B.p[p][i] - V.p[p][i];
+        }
+    }
+}
+
+template <typename T>
+__global__ void hadamard_open_kernel(CPair<T> mE, CPair<T> mF, CPair<T> U, CPair<T> V, CPair<T> Z,
+                                     int64_t n, int trunc, Pair<T> C) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const T e = mE.p[0][i] + mE.p[1][i], f = mF.p[0][i] + mF.p[1][i];
+#pragma unroll
+        for (int p = 0; p < 2; ++p) {
+            T c = (T)p * e * f + e * V.p[p][i] + U.p[p][i] * f + Z.p[p][i];
+            C.p[p][i] = trunc_share<T>(c, p, trunc);
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------------------------
+// Secure MSB chain (R9): Kogge-Stone carry on boolean shares, one kernel per round.
+// Input modes: 0 = x as given (n elements); 1 = Eq. 9 pair [z + h ; z - h] over z of n/2
+// elements (party 0 adds the public +-h, h = 2^(f-1)).
+// State per party: G, P words.  Messages per party: up to 4 words (e, f of two ANDs).
+// ---------------------------------------------------------------------------------------------
+template <typename T>
+struct MsbArgs {
+    CPair<T> x;        // input shares (n, or n/2 in mode 1)
+    CPair<T> mat;      // dealer material
+    Pair<T> G, P;      // state, n words per party
+    Pair<T> msg;       // 4 n words per party
+    int64_t n;
+    int mode;
+    T half;            // 2^(f-1) for mode 1
+    int L, l;
+};
+
+template <typename T>
+__device__ __forceinline__ T msb_input(const MsbArgs<T> &a, int p, int64_t e) {
+    if (a.mode == 0) return a.x.p[p][e];
+    const int64_t h = a.n >> 1;
+    if (e < h) return a.x.p[p][e] + (p == 0 ? a.half : (T)0);
+    return a.x.p[p][e - h] - (p == 0 ? a.half : (T)0);
+}
+
+template <typename T>
+__device__ __forceinline__ const T *mat_ptr(const MsbArgs<T> &a, int p, int t, int w) {
+    return a.mat.p[p] + ((int64_t)t * 3 + w) * a.n;
+}
+
+// Round 1: mask AND t = 0 with X = (x0, 0), Y = (0, x1).
+template <typename T>
+__global__ void msb_round0_kernel(MsbArgs<T> a) {
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < a.n; e += (int64_t)gridDim.x * blockDim.x) {
+#pragma unroll
+        for (int p = 0; p < 2; ++p) {
+            T x = msb_input(a, p, e);
+            T X = p == 0 ? x : (T)0, Y = p == 1 ? x : (T)0;
+            a.msg.p[p][e] = X ^ mat_ptr(a, p, 0, 0)[e];
+            a.msg.p[p][a.n + e] = Y ^ mat_ptr(a, p, 0, 1)[e];
+        }
+    }
+}
+
+// open one AND (message words w, w+1) of AND index t: returns both parties' z.
+template <typename T>
+__device__ __forceinline__ void and_open(const MsbArgs<T> &a, int64_t e, int w, int t, T z[2]) {
+    const T ee = a.msg.p[0][(int64_t)w * a.n + e] ^ a.msg.p[1][(int64_t)w * a.n + e];
+    const T ff = a.msg.p[0][(int64_t)(w + 1) * a.n + e] ^ a.msg.p[1][(int64_t)(w + 1) * a.n + e];
+#pragma unroll
+    for (int p = 0; p < 2; ++p) {
+        T r = (ee & mat_ptr(a, p, t, 1)[e]) ^ (mat_ptr(a, p, t, 0)[e] & ff) ^ mat_ptr(a, p, t, 2)[e];
+        z[p] = p == 1 ? (T)(r ^ (ee & ff)) : r;
+    }
+}
+
+// Round j+1 (j = 1..L): open level j-1's ANDs, update G/P, mask level j's ANDs.
+template <typename T>
+__global__ void msb_level_kernel(MsbArgs<T> a, int j) {
+    const int k = 1 << (j - 1);
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < a.n; e += (int64_t)gridDim.x * blockDim.x) {
+        T G[2], P[2], z[2];
+        if (j == 1) {
+            and_open(a, e, 0, 0, z);
+#pragma unroll
+            for (int p = 0; p < 2; ++p) { G[p] = z[p]; P[p] = msb_input(a, p, e); }
+        } else {
+            and_open(a, e, 0, 2 * j - 3, z);
+            T zp[2];
+            and_open(a, e, 2, 2 * j - 2, zp);
+#pragma unroll
+            for (int p = 0; p < 2; ++p) { G[p] = a.G.p[p][e] ^ z[p]; P[p] = zp[p]; }
+        }
+#pragma unroll
+        for (int p = 0; p < 2; ++p) {
+            const int t1 = 2 * j - 1;
+            a.msg.p[p][e] = P[p] ^ mat_ptr(a, p, t1, 0)[e];
+            a.msg.p[p][a.n + e] = (T)(G[p] << k) ^ mat_ptr(a, p, t1, 1)[e];
+            if (j < a.L) {
+                const int t2 = 2 * j;
+                a.msg.p[p][2 * a.n + e] = P[p] ^ mat_ptr(a, p, t2, 0)[e];
+                a.msg.p[p][3 * a.n + e] = (T)(P[p] << k) ^ mat_ptr(a, p, t2, 1)[e];
+            }
+            a.G.p[p][e] = G[p];
+            a.P.p[p][e] = P[p];
+        }
+    }
+}
+
+// Round L+2: open the last G AND, msb_i = x_i[l-1] ^ G_i[l-2]; emit the B2A message c_i.
+template <typename T>
+__global__ void msb_final_kernel(MsbArgs<T> a, Pair<T> msbB) {
+    const int t = 2 * a.L - 1;
+    const int64_t off = (int64_t)2 * a.L * 3 * a.n;
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < a.n; e += (int64_t)gridDim.x * blockDim.x) {
+        T z[2];
+        and_open(a, e, 0, t, z);
+#pragma unroll
+        for (int p = 0; p < 2; ++p) {
+            T G = a.G.p[p][e] ^ z[p];
+            T x = msb_input(a, p, e);
+            T b = ((x >> (a.l - 1)) & 1) ^ ((G >> (a.l - 2)) & 1);
+            if (msbB.p[p]) msbB.p[p][e] = b;
+            a.msg.p[p][e] = b ^ a.mat.p[p][off + e];   // c_i = msb_i ^ rB_i
+        }
+    }
+}
+
+// Round L+3: open c, [msb]^A; then either store msbA (what = 0) or, for ReLU/Eq. 9 (what = 1),
+// form drelu_i = [i==0] - msbA_i and mask the Hadamard x . drelu (messages mE, mF).
+template <typename T>
+__global__ void msb_b2a_kernel(MsbArgs<T> a, Pair<T> msbA, Pair<T> drelu, CPair<T> U, CPair<T> V,
+                               Pair<T> mE, Pair<T> mF, int what) {
+    const int64_t off = (int64_t)2 * a.L * 3 * a.n;
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < a.n; e += (int64_t)gridDim.x * blockDim.x) {
+        const T c = a.msg.p[0][e] ^ a.msg.p[1][e];
+        const T s = (T)1 - (T)2 * c;
+#pragma unroll
+        for (int p = 0; p < 2; ++p) {
+            T m = (p == 0 ? c : (T)0) + s * a.mat.p[p][off + a.n + e];
+            if (what == 0) {
+                msbA.p[p][e] = m;
+            } else {
+                T d = (p == 0 ? (T)1 : (T)0) - m;
+                if (drelu.p[p]) drelu.p[p][e] = d;
+                mE.p[p][e] = msb_input(a, p, e) - U.p[p][e];
+                mF.p[p][e] = d - V.p[p][e];
+            }
+        }
+    }
+}
+
+// Round L+4 for Eq. 9: open the Hadamard of 2n' elements, y_i = r_i[e] - r_i[e + n'].
+template <typename T>
+__global__ void eq9_open_kernel(CPair<T> mE, CPair<T> mF, CPair<T> U, CPair<T> V, CPair<T> Z,
+                                int64_t nh, Pair<T> y, CPair<T> Ysub, Pair<T> delta) {
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < nh; e += (int64_t)gridDim.x * blockDim.x) {
+        const T e1 = mE.p[0][e] + mE.p[1][e], f1 = mF.p[0][e] + mF.p[1][e];
+        const T e2 = mE.p[0][e + nh] + mE.p[1][e + nh], f2 = mF.p[0][e + nh] + mF.p[1][e + nh];
+#pragma unroll
+        for (int p = 0; p < 2; ++p) {
+            T r1 = (T)p * e1 * f1 + e1 * V.p[p][e] + U.p[p][e] * f1 + Z.p[p][e];
+            T r2 = (T)p * e2 * f2 + e2 * V.p[p][e + nh] + U.p[p][e + nh] * f2 + Z.p[p][e + nh];
+            T out = r1 - r2;
+            if (y.p[p]) y.p[p][e] = out;
+            if (delta.p[p]) delta.p[p][e] = out - Ysub.p[p][e];
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------------------------
+// training helpers
+// ---------------------------------------------------------------------------------------------
+template <typename T>
+__global__ void sub_pair_kernel(CPair<T> a, CPair<T> b, int64_t n, Pair<T> c) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        c.p[0][i] = a.p[0][i] - b.p[0][i];
+        c.p[1][i] = a.p[1][i] - b.p[1][i];
+    }
+}
+
+// W^m_i -= trunc_i(g_i, s_grad); W_i = trunc_i(W^m_i, s_fwd)   (R14)
+template <typename T>
+__global__ void update_kernel(Pair<T> Wm, Pair<T> W, CPair<T> g, int64_t n, int s_grad, int s_fwd) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+#pragma unroll
+        for (int p = 0; p < 2; ++p) {
+            T wm = Wm.p[p][i] - trunc_share<T>(g.p[p][i], p, s_grad);
+            Wm.p[p][i] = wm;
+            W.p[p][i] = trunc_share<T>(wm, p, s_fwd);
+        }
+    }
+}
+
+template <typename T>
+__global__ void truncate_pair_kernel(CPair<T> src, Pair<T> dst, int64_t n, int d) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        dst.p[0][i] = trunc_share<T>(src.p[0][i], 0, d);
+        dst.p[1][i] = trunc_share<T>(src.p[1][i], 1, d);
+    }
+}
+
+}  // namespace psml

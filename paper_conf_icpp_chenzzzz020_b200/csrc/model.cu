@@ -1,0 +1,568 @@
+// model.cu -- secure training / inference of linear & logistic regression, MLP and CNN on the
+// co-resident pair engine (Sec. 4.3 "Detailed Design" L201-L207; Sec. 7.1).
+//
+// One step (per pair, batch B rows), all in Z_{2^64} with f = 13 fractional bits:
+//   forward   z_l = trunc(h_l . W_l)            Beaver matmul (op 0)
+//             h_{l+1} = ReLU(z_l)  (hidden)      MSB chain + Hadamard (ops 3, 6/0), keeps DReLU
+//             yhat = Eq. 9(z_L) (logistic/MLP/CNN) or z_L (linear)   (ops 4, 6/2)
+//   backward  delta = yhat - y
+//             gW_l = h_l^T . delta               Beaver matmul, untruncated (op 1)
+//             delta = trunc(delta . W_l^T) (.) DReLU_{l-1}   (op 2, Hadamard 6/1)
+//   update    W^m_l -= trunc(gW_l, 26 + s_lr - m); W_l = trunc(W^m_l, m - f)   (R14)
+// Every triplet / MSB material comes from the model's dealer pool filled by psml_model_deal with
+// call id (pair, step, layer, op, slot) -- identical to oracle/protocol.py (R11).
+#include <cstring>
+#include <memory>
+#include <string>
+#include <vector>
+
+#include "engine.h"
+
+namespace psml {
+
+using T = uint64_t;
+
+enum { OP_FWD = 0, OP_GRADW = 1, OP_GRADIN = 2, OP_RELU_MSB = 3, OP_EQ9_MSB = 4, OP_HADAMARD = 6 };
+enum ItemKind { IT_MATRIX, IT_CONV_FWD, IT_CONV_GW, IT_HAD, IT_MSB };
+
+static inline uint64_t call_id(uint32_t pair, uint32_t step, int layer, int op, int slot) {
+    return ((uint64_t)(pair & 0xFF) << 56) | ((uint64_t)step << 24) | ((uint64_t)(layer & 0xFF) << 16) |
+           ((uint64_t)(op & 0xFF) << 8) | (uint64_t)(slot & 0xFF);
+}
+
+struct Buf {  // a pair of device buffers of `n` words
+    T *p[2] = {nullptr, nullptr};
+    int64_t n = 0;
+    T *const *pp() { return p; }
+    const T *const *cp() const { return (const T *const *)p; }
+};
+
+struct DealItem {
+    ItemKind kind;
+    int layer, op, slot;
+    int64_t M = 0, K = 0, N = 0, n = 0;
+    bool fwd = true;  // needed by inference
+    Buf U, V, Z, mat;
+};
+
+}  // namespace psml
+
+struct psml_model_s {
+    psml::Ctx *ctx = nullptr;
+    psml_model_desc d{};
+    int nl = 0;
+    int64_t B = 0;
+    std::vector<int64_t> rows, cols;  // weight shapes
+    std::vector<int64_t> dims;        // MLP-style widths d_0..d_L (CNN: d_1 = 12544 after conv)
+    psml::ConvGeom g{};
+    std::vector<psml::Buf> Wm, W;
+    psml::T *grad_base = nullptr;
+    int64_t grad_words = 0;
+    std::vector<int64_t> grad_off;
+    // activations
+    std::vector<psml::Buf> act, z, drelu;  // act[l]: input of layer l (l >= 1 model-owned)
+    psml::Buf yhat, delta, tmp;
+    std::vector<psml::DealItem> items;
+    psml::T *ws = nullptr;
+    int64_t ws_words = 0;
+    std::vector<void *> allocs;
+    int64_t dealt_step = -1;
+    bool dealt_full = false;
+    bool grads_ready = false;
+};
+
+namespace psml {
+
+static psml_status dalloc(psml_model_s *m, T **out, int64_t words) {
+    if (words <= 0) { *out = nullptr; return PSML_OK; }
+    void *p = nullptr;
+    if (cudaMalloc(&p, sizeof(T) * (size_t)words) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(PSML_ERR_NOMEM, "model allocation of " + std::to_string(words * 8) + " bytes failed");
+    }
+    m->allocs.push_back(p);
+    *out = (T *)p;
+    return PSML_OK;
+}
+
+static psml_status balloc(psml_model_s *m, Buf &b, int64_t n) {
+    b.n = n;
+    PSML_TRY(dalloc(m, &b.p[0], n));
+    return dalloc(m, &b.p[1], n);
+}
+
+static DealItem *find_item(psml_model_s *m, int layer, int op, int slot) {
+    for (auto &it : m->items)
+        if (it.layer == layer && it.op == op && it.slot == slot) return &it;
+    return nullptr;
+}
+
+static void add_matrix(psml_model_s *m, int layer, int op, int64_t M, int64_t K, int64_t N, bool fwd) {
+    DealItem it;
+    it.kind = IT_MATRIX; it.layer = layer; it.op = op; it.slot = 0; it.M = M; it.K = K; it.N = N; it.fwd = fwd;
+    m->items.push_back(it);
+}
+static void add_had(psml_model_s *m, int layer, int slot, int64_t n, bool fwd) {
+    DealItem it;
+    it.kind = IT_HAD; it.layer = layer; it.op = OP_HADAMARD; it.slot = slot; it.n = n; it.fwd = fwd;
+    m->items.push_back(it);
+}
+static void add_msb(psml_model_s *m, int layer, int op, int64_t n, bool fwd) {
+    DealItem it;
+    it.kind = IT_MSB; it.layer = layer; it.op = op; it.slot = 0; it.n = n; it.fwd = fwd;
+    m->items.push_back(it);
+}
+
+static bool is_eq9_out(const psml_model_s *m) { return m->d.kind != PSML_LINREG; }
+
+static void plan_items(psml_model_s *m) {
+    const int64_t B = m->B;
+    if (m->d.kind == PSML_CNN) {
+        const ConvGeom &g = m->g;
+        const int64_t rows = B * g.OH * g.OW, kk = (int64_t)g.C * g.k * g.k;
+        const int64_t h1 = m->dims[1], hid = m->dims[2], cls = m->dims[3];
+        DealItem cf;
+        cf.kind = IT_CONV_FWD; cf.layer = 0; cf.op = OP_FWD; cf.slot = 0;
+        cf.M = rows; cf.K = kk; cf.N = m->cols[0]; cf.fwd = true;
+        m->items.push_back(cf);
+        add_msb(m, 0, OP_RELU_MSB, B * h1, true);
+        add_had(m, 0, 0, B * h1, true);
+        add_matrix(m, 1, OP_FWD, B, h1, hid, true);
+        add_msb(m, 1, OP_RELU_MSB, B * hid, true);
+        add_had(m, 1, 0, B * hid, true);
+        add_matrix(m, 2, OP_FWD, B, hid, cls, true);
+        add_msb(m, 2, OP_EQ9_MSB, 2 * B * cls, true);
+        add_had(m, 2, 2, 2 * B * cls, true);
+        add_matrix(m, 2, OP_GRADW, hid, B, cls, false);
+        add_matrix(m, 2, OP_GRADIN, B, cls, hid, false);
+        add_had(m, 1, 1, B * hid, false);
+        add_matrix(m, 1, OP_GRADW, h1, B, hid, false);
+        add_matrix(m, 1, OP_GRADIN, B, hid, h1, false);
+        add_had(m, 0, 1, B * h1, false);
+        DealItem cg;
+        cg.kind = IT_CONV_GW; cg.layer = 0; cg.op = OP_GRADW; cg.slot = 0;
+        cg.M = kk; cg.K = rows; cg.N = m->cols[0]; cg.fwd = false;
+        m->items.push_back(cg);
+        return;
+    }
+    const int nl = m->nl;
+    for (int l = 0; l < nl; ++l) {
+        add_matrix(m, l, OP_FWD, B, m->dims[l], m->dims[l + 1], true);
+        const int64_t n = B * m->dims[l + 1];
+        if (l < nl - 1) {
+            add_msb(m, l, OP_RELU_MSB, n, true);
+            add_had(m, l, 0, n, true);
+        } else if (is_eq9_out(m)) {
+            add_msb(m, l, OP_EQ9_MSB, 2 * n, true);
+            add_had(m, l, 2, 2 * n, true);
+        }
+    }
+    for (int l = nl - 1; l >= 0; --l) {
+        add_matrix(m, l, OP_GRADW, m->dims[l], B, m->dims[l + 1], false);
+        if (l > 0) {
+            add_matrix(m, l, OP_GRADIN, B, m->dims[l + 1], m->dims[l], false);
+            add_had(m, l - 1, 1, B * m->dims[l], false);
+        }
+    }
+}
+
+static psml_status alloc_items(psml_model_s *m) {
+    const psml_ring ring = m->ctx->ring;
+    for (auto &it : m->items) {
+        switch (it.kind) {
+        case IT_MATRIX:
+            PSML_TRY(balloc(m, it.U, it.M * it.K));
+            PSML_TRY(balloc(m, it.V, it.K * it.N));
+            PSML_TRY(balloc(m, it.Z, it.M * it.N));
+            break;
+        case IT_CONV_FWD:
+        case IT_CONV_GW: {
+            const int64_t nin = m->B * m->g.C * m->g.H * m->g.W;
+            PSML_TRY(balloc(m, it.U, nin));
+            PSML_TRY(balloc(m, it.V, it.K * it.N));
+            PSML_TRY(balloc(m, it.Z, it.M * it.N));
+            break;
+        }
+        case IT_HAD:
+            PSML_TRY(balloc(m, it.U, it.n));
+            PSML_TRY(balloc(m, it.V, it.n));
+            PSML_TRY(balloc(m, it.Z, it.n));
+            break;
+        case IT_MSB:
+            PSML_TRY(balloc(m, it.mat, psml_msb_material_words(ring, it.n)));
+            break;
+        }
+    }
+    return PSML_OK;
+}
+
+static int64_t ws_need(psml_model_s *m) {
+    int64_t w = 0;
+    for (auto &it : m->items) {
+        switch (it.kind) {
+        case IT_MATRIX: w = std::max(w, beaver_ws_words<T>(it.M, it.K, it.N)); break;
+        case IT_CONV_FWD: w = std::max(w, conv_ws_words<T>(m->B, m->g, 0, it.N)); break;
+        case IT_CONV_GW: w = std::max(w, conv_ws_words<T>(m->B, m->g, 1, it.N)); break;
+        case IT_HAD: w = std::max(w, 4 * it.n); break;
+        case IT_MSB: w = std::max(w, msb_ws_words<T>(it.n)); break;
+        }
+    }
+    // dealer: conv Z GEMM split-K partials + plain triplet partials
+    for (auto &it : m->items)
+        if (it.kind != IT_HAD && it.kind != IT_MSB) w = std::max(w, it.M * it.N);
+    return w;
+}
+
+// ------------------------------------------------------------------------------------------------
+// dealer (offline phase)
+// ------------------------------------------------------------------------------------------------
+static psml_status deal_item(psml_model_s *m, DealItem &it, uint32_t step, cudaStream_t s) {
+    const uint64_t seed = m->d.dealer_seed;
+    const uint64_t cid = call_id(m->d.pair_id, step, it.layer, it.op, it.slot);
+    switch (it.kind) {
+    case IT_MATRIX: {
+        dealer_pair_kernel<T><<<grid_for(it.M * it.K / 8 + 1, 256), 256, 0, s>>>(
+            make_key(seed, TAG_U0, cid), make_key(seed, TAG_U1, cid), it.M * it.K, it.U.p[0], it.U.p[1], nullptr);
+        PSML_LAUNCH_CHECK();
+        dealer_pair_kernel<T><<<grid_for(it.K * it.N / 8 + 1, 256), 256, 0, s>>>(
+            make_key(seed, TAG_V0, cid), make_key(seed, TAG_V1, cid), it.K * it.N, it.V.p[0], it.V.p[1], nullptr);
+        PSML_LAUNCH_CHECK();
+        DealerOps<T> ops;
+        ops.U0 = it.U.p[0]; ops.U1 = it.U.p[1]; ops.V0 = it.V.p[0]; ops.V1 = it.V.p[1];
+        ops.Z0 = it.Z.p[0]; ops.Z1 = it.Z.p[1]; ops.kz0 = make_key(seed, TAG_Z0, cid);
+        ops.M = it.M; ops.N = it.N; ops.Kext = it.K;
+        return launch_ring_gemm<T, DealerOps<T>>(ops, m->ws, m->ws_words, s, m->ctx->sm_count);
+    }
+    case IT_CONV_FWD:
+    case IT_CONV_GW: {
+        const int64_t nin = it.U.n;
+        dealer_pair_kernel<T><<<grid_for(nin / 8 + 1, 256), 256, 0, s>>>(
+            make_key(seed, TAG_U0, cid), make_key(seed, TAG_U1, cid), nin, it.U.p[0], it.U.p[1], nullptr);
+        PSML_LAUNCH_CHECK();
+        dealer_pair_kernel<T><<<grid_for(it.K * it.N / 8 + 1, 256), 256, 0, s>>>(
+            make_key(seed, TAG_V0, cid), make_key(seed, TAG_V1, cid), it.K * it.N, it.V.p[0], it.V.p[1], nullptr);
+        PSML_LAUNCH_CHECK();
+        ConvDealerOps<T> ops;
+        ops.U0 = it.U.p[0]; ops.U1 = it.U.p[1]; ops.V0 = it.V.p[0]; ops.V1 = it.V.p[1];
+        ops.Z0 = it.Z.p[0]; ops.Z1 = it.Z.p[1]; ops.kz0 = make_key(seed, TAG_Z0, cid);
+        ops.g = m->g; ops.M = it.M; ops.N = it.N; ops.Kext = it.K; ops.transposed = it.kind == IT_CONV_GW;
+        return launch_ring_gemm<T, ConvDealerOps<T>>(ops, m->ws, m->ws_words, s, m->ctx->sm_count);
+    }
+    case IT_HAD: {
+        void *U[2] = {it.U.p[0], it.U.p[1]}, *V[2] = {it.V.p[0], it.V.p[1]}, *Z[2] = {it.Z.p[0], it.Z.p[1]};
+        return hadamard_triplet_launch<T>(seed, cid, it.n, U, V, Z, s);
+    }
+    case IT_MSB: {
+        void *mt[2] = {it.mat.p[0], it.mat.p[1]};
+        return msb_dealer_launch<T>(seed, cid, it.n, mt, s);
+    }
+    }
+    return PSML_OK;
+}
+
+// ------------------------------------------------------------------------------------------------
+// online pieces
+// ------------------------------------------------------------------------------------------------
+static psml_status mm(psml_model_s *m, const T *const A[2], const T *const Bm[2], int layer, int op, int flags,
+                      int trunc, T *const C[2], cudaStream_t s) {
+    DealItem *it = find_item(m, layer, op, 0);
+    if (!it) return fail(PSML_ERR_STATE, "missing triplet");
+    return beaver_matmul<T>(A, Bm, it->U.cp(), it->V.cp(), it->Z.cp(), it->M, it->K, it->N, flags, trunc, C, m->ws,
+                            m->ws_words, s, m->ctx->sm_count);
+}
+
+static psml_status relu(psml_model_s *m, const T *const x[2], int layer, T *const y[2], T *const dr[2],
+                        cudaStream_t s) {
+    DealItem *mat = find_item(m, layer, OP_RELU_MSB, 0), *h = find_item(m, layer, OP_HADAMARD, 0);
+    if (!mat || !h) return fail(PSML_ERR_STATE, "missing ReLU material");
+    return msb_chain<T>(x, mat->n, mat->mat.cp(), 0, 0, 1, nullptr, nullptr, dr, h->U.cp(), h->V.cp(), h->Z.cp(), y,
+                        nullptr, nullptr, m->ws, s);
+}
+
+static psml_status eq9(psml_model_s *m, const T *const z[2], int layer, T *const y[2], const T *const Y[2],
+                       T *const dlt[2], cudaStream_t s) {
+    DealItem *mat = find_item(m, layer, OP_EQ9_MSB, 0), *h = find_item(m, layer, OP_HADAMARD, 2);
+    if (!mat || !h) return fail(PSML_ERR_STATE, "missing Eq. 9 material");
+    const T half = (T)1 << (m->ctx->ring.frac_bits - 1);
+    return msb_chain<T>(z, mat->n, mat->mat.cp(), 1, half, 2, nullptr, nullptr, nullptr, h->U.cp(), h->V.cp(),
+                        h->Z.cp(), y, Y, dlt, m->ws, s);
+}
+
+static psml_status had(psml_model_s *m, const T *const a[2], const T *const b[2], int layer, int slot, T *const c[2],
+                       cudaStream_t s) {
+    DealItem *h = find_item(m, layer, OP_HADAMARD, slot);
+    if (!h) return fail(PSML_ERR_STATE, "missing Hadamard triplet");
+    return beaver_hadamard<T>(a, b, h->U.cp(), h->V.cp(), h->Z.cp(), h->n, 0, c, m->ws, s);
+}
+
+static psml_status sub(const T *const a[2], const T *const b[2], int64_t n, T *const c[2], cudaStream_t s) {
+    sub_pair_kernel<T><<<ew_grid(n), EW_THREADS, 0, s>>>(CPair<T>{{a[0], a[1]}}, CPair<T>{{b[0], b[1]}}, n,
+                                                          Pair<T>{{c[0], c[1]}});
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
+static psml_status conv(psml_model_s *m, const T *const X[2], const T *const Bm[2], int transposed, int trunc,
+                        T *const C[2], cudaStream_t s) {
+    DealItem *it = find_item(m, 0, transposed ? OP_GRADW : OP_FWD, 0);
+    if (!it) return fail(PSML_ERR_STATE, "missing conv triplet");
+    return conv_beaver<T>(X, Bm, it->U.cp(), it->V.cp(), it->Z.cp(), m->B, m->g, transposed, it->N, trunc, C, m->ws,
+                          m->ws_words, s, m->ctx->sm_count);
+}
+
+static T *const *gradp(psml_model_s *m, int layer, T *tmp[2]) {
+    tmp[0] = m->grad_base + m->grad_off[layer];
+    tmp[1] = m->grad_base + m->grad_words + m->grad_off[layer];
+    return tmp;
+}
+
+// forward pass; if Y != nullptr also leaves delta = yhat - Y in m->delta
+static psml_status forward(psml_model_s *m, const T *const X[2], const T *const Y[2], T *const out[2],
+                           cudaStream_t s) {
+    const int F = m->ctx->ring.frac_bits;
+    m->act[0].p[0] = (T *)X[0];
+    m->act[0].p[1] = (T *)X[1];
+    T *yo[2] = {out ? out[0] : m->yhat.p[0], out ? out[1] : m->yhat.p[1]};
+    if (m->d.kind == PSML_CNN) {
+        PSML_TRY(conv(m, X, m->W[0].cp(), 0, F, m->z[0].pp(), s));
+        PSML_TRY(relu(m, m->z[0].cp(), 0, m->act[1].pp(), m->drelu[0].pp(), s));
+        PSML_TRY(mm(m, m->act[1].cp(), m->W[1].cp(), 1, OP_FWD, 0, F, m->z[1].pp(), s));
+        PSML_TRY(relu(m, m->z[1].cp(), 1, m->act[2].pp(), m->drelu[1].pp(), s));
+        PSML_TRY(mm(m, m->act[2].cp(), m->W[2].cp(), 2, OP_FWD, 0, F, m->z[2].pp(), s));
+        return eq9(m, m->z[2].cp(), 2, yo, Y, Y ? m->delta.pp() : nullptr, s);
+    }
+    const int nl = m->nl;
+    for (int l = 0; l < nl; ++l) {
+        PSML_TRY(mm(m, m->act[l].cp(), m->W[l].cp(), l, OP_FWD, 0, F, m->z[l].pp(), s));
+        if (l < nl - 1) {
+            PSML_TRY(relu(m, m->z[l].cp(), l, m->act[l + 1].pp(), m->drelu[l].pp(), s));
+        } else if (is_eq9_out(m)) {
+            PSML_TRY(eq9(m, m->z[l].cp(), l, yo, Y, Y ? m->delta.pp() : nullptr, s));
+        } else {
+            const int64_t n = m->B * m->dims[nl];
+            for (int p = 0; p < 2; ++p)
+                PSML_CUDA_TRY(cudaMemcpyAsync(yo[p], m->z[l].p[p], sizeof(T) * n, cudaMemcpyDeviceToDevice, s));
+            if (Y) PSML_TRY(sub(m->z[l].cp(), Y, n, m->delta.pp(), s));
+        }
+    }
+    return PSML_OK;
+}
+
+static psml_status backward(psml_model_s *m, cudaStream_t s) {
+    const int F = m->ctx->ring.frac_bits;
+    T *g[2];
+    if (m->d.kind == PSML_CNN) {
+        // layer 2 (FC 64 -> 10)
+        PSML_TRY(mm(m, m->act[2].cp(), m->delta.cp(), 2, OP_GRADW, PSML_TRANS_A, 0, gradp(m, 2, g), s));
+        PSML_TRY(mm(m, m->delta.cp(), m->W[2].cp(), 2, OP_GRADIN, PSML_TRANS_B, F, m->tmp.pp(), s));
+        PSML_TRY(had(m, m->tmp.cp(), m->drelu[1].cp(), 1, 1, m->delta.pp(), s));
+        // layer 1 (FC 12544 -> 64)
+        PSML_TRY(mm(m, m->act[1].cp(), m->delta.cp(), 1, OP_GRADW, PSML_TRANS_A, 0, gradp(m, 1, g), s));
+        PSML_TRY(mm(m, m->delta.cp(), m->W[1].cp(), 1, OP_GRADIN, PSML_TRANS_B, F, m->tmp.pp(), s));
+        PSML_TRY(had(m, m->tmp.cp(), m->drelu[0].cp(), 0, 1, m->delta.pp(), s));
+        // conv weight gradient: im2col(X)^T . delta   (delta viewed as (B*OH*OW) x Cout)
+        return conv(m, m->act[0].cp(), m->delta.cp(), 1, 0, gradp(m, 0, g), s);
+    }
+    const int nl = m->nl;
+    for (int l = nl - 1; l >= 0; --l) {
+        PSML_TRY(mm(m, m->act[l].cp(), m->delta.cp(), l, OP_GRADW, PSML_TRANS_A, 0, gradp(m, l, g), s));
+        if (l > 0) {
+            PSML_TRY(mm(m, m->delta.cp(), m->W[l].cp(), l, OP_GRADIN, PSML_TRANS_B, F, m->tmp.pp(), s));
+            PSML_TRY(had(m, m->tmp.cp(), m->drelu[l - 1].cp(), l - 1, 1, m->delta.pp(), s));
+        }
+    }
+    return PSML_OK;
+}
+
+}  // namespace psml
+
+using namespace psml;
+
+// ABI definitions: C linkage and default visibility come from include/psml.h.
+
+psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_model *out) {
+    if (!ctx || !desc || !out) return fail(PSML_ERR_INVALID, "null argument");
+    Ctx *c = reinterpret_cast<Ctx *>(ctx);
+    if (c->ring.l != 64) return fail(PSML_ERR_UNSUPPORTED, "training models run in Z_2^64 (DESIGN.md R18)");
+    if (desc->batch <= 0) return fail(PSML_ERR_SHAPE, "batch must be positive");
+    if (desc->master_frac_bits < c->ring.frac_bits || desc->lr_shift < 0)
+        return fail(PSML_ERR_INVALID, "master_frac_bits must be >= frac_bits and lr_shift >= 0");
+    if (2 * c->ring.frac_bits + desc->lr_shift - desc->master_frac_bits < 0)
+        return fail(PSML_ERR_INVALID, "2f + lr_shift - m must be >= 0");
+    std::unique_ptr<psml_model_s> m(new psml_model_s());
+    m->ctx = c;
+    m->d = *desc;
+    m->B = desc->batch;
+    switch (desc->kind) {
+    case PSML_LINREG:
+    case PSML_LOGREG:
+    case PSML_MLP: {
+        int nl = desc->n_layers;
+        if (desc->kind != PSML_MLP) nl = 1;
+        if (nl < 1 || nl > 7) return fail(PSML_ERR_SHAPE, "n_layers must be in [1, 7]");
+        for (int i = 0; i <= nl; ++i)
+            if (desc->dims[i] <= 0) return fail(PSML_ERR_SHAPE, "dims must be positive");
+        m->nl = nl;
+        for (int i = 0; i <= nl; ++i) m->dims.push_back(desc->dims[i]);
+        for (int l = 0; l < nl; ++l) { m->rows.push_back(m->dims[l]); m->cols.push_back(m->dims[l + 1]); }
+        break;
+    }
+    case PSML_CNN: {
+        ConvGeom g;
+        g.C = desc->cnn_c; g.H = desc->cnn_h; g.W = desc->cnn_w; g.k = desc->cnn_k;
+        if (g.C <= 0 || g.k <= 0 || g.H < g.k || g.W < g.k || desc->cnn_cout <= 0 || desc->cnn_cout > 16 ||
+            desc->cnn_hidden <= 0 || desc->cnn_classes <= 0)
+            return fail(PSML_ERR_SHAPE, "bad CNN geometry (cout must be <= 16)");
+        g.OH = g.H - g.k + 1; g.OW = g.W - g.k + 1;
+        m->g = g;
+        m->nl = 3;
+        const int64_t flat = (int64_t)g.OH * g.OW * desc->cnn_cout;
+        m->dims = {(int64_t)g.C * g.H * g.W, flat, desc->cnn_hidden, desc->cnn_classes};
+        m->rows = {(int64_t)g.C * g.k * g.k, flat, desc->cnn_hidden};
+        m->cols = {desc->cnn_cout, desc->cnn_hidden, desc->cnn_classes};
+        break;
+    }
+    default:
+        return fail(PSML_ERR_INVALID, "unknown model kind");
+    }
+    psml_model_s *mp = m.get();
+    int64_t tot = 0;
+    for (int l = 0; l < m->nl; ++l) {
+        Buf b;
+        PSML_TRY(balloc(mp, b, m->rows[l] * m->cols[l]));
+        m->Wm.push_back(b);
+        PSML_TRY(balloc(mp, b, m->rows[l] * m->cols[l]));
+        m->W.push_back(b);
+        m->grad_off.push_back(tot);
+        tot += m->rows[l] * m->cols[l];
+    }
+    m->grad_words = tot;
+    PSML_TRY(dalloc(mp, &m->grad_base, 2 * tot));
+    const int64_t B = m->B;
+    m->act.resize(m->nl);
+    m->z.resize(m->nl);
+    m->drelu.resize(m->nl);
+    int64_t maxw = 0;
+    for (int l = 0; l < m->nl; ++l) {
+        if (l >= 1) PSML_TRY(balloc(mp, m->act[l], B * m->dims[l]));
+        const int64_t zn = B * m->dims[l + 1];
+        PSML_TRY(balloc(mp, m->z[l], zn));
+        if (l < m->nl - 1) PSML_TRY(balloc(mp, m->drelu[l], zn));
+        maxw = std::max(maxw, std::max(m->dims[l + 1], l >= 1 ? m->dims[l] : (int64_t)0));
+    }
+    PSML_TRY(balloc(mp, m->yhat, B * m->dims[m->nl]));
+    PSML_TRY(balloc(mp, m->delta, B * maxw));
+    PSML_TRY(balloc(mp, m->tmp, B * maxw));
+    plan_items(mp);
+    PSML_TRY(alloc_items(mp));
+    m->ws_words = ws_need(mp);
+    PSML_TRY(dalloc(mp, &m->ws, m->ws_words));
+    *out = m.release();
+    return PSML_OK;
+}
+
+psml_status psml_model_destroy(psml_model model) {
+    if (!model) return PSML_OK;
+    cudaDeviceSynchronize();
+    for (void *p : model->allocs) cudaFree(p);
+    delete model;
+    return PSML_OK;
+}
+
+psml_status psml_model_layer_shape(psml_model m, int32_t layer, int64_t *rows, int64_t *cols) {
+    if (!m || layer < 0 || layer >= m->nl) return fail(PSML_ERR_INVALID, "bad model or layer");
+    if (rows) *rows = m->rows[layer];
+    if (cols) *cols = m->cols[layer];
+    return PSML_OK;
+}
+
+psml_status psml_model_set_master(psml_model m, int32_t layer, const void *const Wm[2], psml_stream stream) {
+    if (!m || layer < 0 || layer >= m->nl || !Wm) return fail(PSML_ERR_INVALID, "bad model, layer or pointer");
+    PSML_TRY(check_ptrs({Wm[0], Wm[1]}));
+    cudaStream_t s = (cudaStream_t)stream;
+    const int64_t n = m->rows[layer] * m->cols[layer];
+    for (int p = 0; p < 2; ++p)
+        PSML_CUDA_TRY(cudaMemcpyAsync(m->Wm[layer].p[p], Wm[p], sizeof(T) * n, cudaMemcpyDeviceToDevice, s));
+    const int sh = m->d.master_frac_bits - m->ctx->ring.frac_bits;
+    truncate_pair_kernel<T><<<ew_grid(n), EW_THREADS, 0, s>>>(CPair<T>{{m->Wm[layer].p[0], m->Wm[layer].p[1]}},
+                                                               Pair<T>{{m->W[layer].p[0], m->W[layer].p[1]}}, n, sh);
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
+psml_status psml_model_get_master(psml_model m, int32_t layer, void *const Wm[2], psml_stream stream) {
+    if (!m || layer < 0 || layer >= m->nl || !Wm) return fail(PSML_ERR_INVALID, "bad model, layer or pointer");
+    PSML_TRY(check_ptrs({Wm[0], Wm[1]}));
+    const int64_t n = m->rows[layer] * m->cols[layer];
+    for (int p = 0; p < 2; ++p)
+        PSML_CUDA_TRY(cudaMemcpyAsync(Wm[p], m->Wm[layer].p[p], sizeof(T) * n, cudaMemcpyDeviceToDevice, (cudaStream_t)stream));
+    return PSML_OK;
+}
+
+psml_status psml_model_deal(psml_model m, uint32_t step_id, int32_t infer_only, psml_stream stream) {
+    if (!m) return fail(PSML_ERR_INVALID, "model is null");
+    cudaStream_t s = (cudaStream_t)stream;
+    for (auto &it : m->items) {
+        if (infer_only && !it.fwd) continue;
+        PSML_TRY(deal_item(m, it, step_id, s));
+    }
+    m->dealt_step = step_id;
+    m->dealt_full = !infer_only;
+    return PSML_OK;
+}
+
+psml_status psml_train_forward_backward(psml_model m, const void *const X[2], const void *const Y[2], uint32_t step_id,
+                                        psml_stream stream) {
+    if (!m || !X || !Y) return fail(PSML_ERR_INVALID, "null argument");
+    PSML_TRY(check_ptrs({X[0], X[1], Y[0], Y[1]}));
+    if (m->dealt_step != (int64_t)step_id || !m->dealt_full)
+        return fail(PSML_ERR_STATE, "psml_model_deal(step_id, infer_only=0) must precede the step");
+    cudaStream_t s = (cudaStream_t)stream;
+    PSML_TRY(forward(m, (const T *const *)X, (const T *const *)Y, nullptr, s));
+    PSML_TRY(backward(m, s));
+    m->grads_ready = true;
+    return PSML_OK;
+}
+
+psml_status psml_model_grads(psml_model m, void **grads, int64_t *words_per_party) {
+    if (!m) return fail(PSML_ERR_INVALID, "model is null");
+    if (grads) *grads = m->grad_base;
+    if (words_per_party) *words_per_party = m->grad_words;
+    return PSML_OK;
+}
+
+psml_status psml_train_apply_update(psml_model m, int32_t extra_shift, psml_stream stream) {
+    if (!m) return fail(PSML_ERR_INVALID, "model is null");
+    if (extra_shift < 0 || extra_shift > 16) return fail(PSML_ERR_INVALID, "extra_shift out of range");
+    if (!m->grads_ready) return fail(PSML_ERR_STATE, "no gradients: run psml_train_forward_backward first");
+    cudaStream_t s = (cudaStream_t)stream;
+    const int f = m->ctx->ring.frac_bits;
+    const int s_grad = 2 * f + m->d.lr_shift - m->d.master_frac_bits + extra_shift;
+    const int s_fwd = m->d.master_frac_bits - f;
+    for (int l = 0; l < m->nl; ++l) {
+        const int64_t n = m->rows[l] * m->cols[l];
+        T *g[2];
+        gradp(m, l, g);
+        update_kernel<T><<<ew_grid(n), EW_THREADS, 0, s>>>(Pair<T>{{m->Wm[l].p[0], m->Wm[l].p[1]}},
+                                                            Pair<T>{{m->W[l].p[0], m->W[l].p[1]}},
+                                                            CPair<T>{{g[0], g[1]}}, n, s_grad, s_fwd);
+        PSML_LAUNCH_CHECK();
+    }
+    m->grads_ready = false;
+    return PSML_OK;
+}
+
+psml_status psml_secure_train_step(psml_model m, const void *const X[2], const void *const Y[2], uint32_t step_id,
+                                   psml_stream stream) {
+    PSML_TRY(psml_train_forward_backward(m, X, Y, step_id, stream));
+    return psml_train_apply_update(m, 0, stream);
+}
+
+psml_status psml_secure_infer(psml_model m, const void *const X[2], uint32_t step_id, void *const Yhat[2],
+                              psml_stream stream) {
+    if (!m || !X || !Yhat) return fail(PSML_ERR_INVALID, "null argument");
+    PSML_TRY(check_ptrs({X[0], X[1], Yhat[0], Yhat[1]}));
+    if (m->dealt_step != (int64_t)step_id) return fail(PSML_ERR_STATE, "psml_model_deal(step_id) must precede inference");
+    return forward(m, (const T *const *)X, nullptr, (T *const *)Yhat, (cudaStream_t)stream);
+}
+

@@ -1,0 +1,180 @@
+// ops.cuh -- host-side building blocks of the co-resident pair engine (shared by engine.cu).
+// Each op = the sequence of round kernels of one protocol step, with explicit workspaces so a
+// model step allocates nothing (and can be captured in a CUDA graph).
+#pragma once
+#include <algorithm>
+
+#include "common.cuh"
+#include "gemm_simt.cuh"
+#include "kernels.cuh"
+
+namespace psml {
+
+constexpr int EW_THREADS = 256;
+
+inline int ew_grid(int64_t n) { return grid_for(n, EW_THREADS, 148 * 32); }
+
+// Tensor-core limb GEMM entry (gemm_tc.cu).  Returns PSML_ERR_UNSUPPORTED when the shape or
+// device does not take the tcgen05 path (the caller then uses the CUDA-core kernels).
+struct TcBeaverArgs;
+psml_status tc_ring_gemm_plain(int l, const void *A, const void *B, int64_t M, int64_t K, int64_t N,
+                               void *C, void *ws, size_t ws_bytes, cudaStream_t s);
+size_t tc_ring_gemm_ws_bytes(int l, int64_t M, int64_t K, int64_t N);
+bool tc_available();
+
+// ---------------------------------------------------------------------------------------------
+// Beaver matmul: mask round (Eq. 4) + fused open/Eq. 8 GEMM/epilogue round.
+// ws_words needs: M*K*2 + K*N*2 (messages) + 2*M*N (split-K partials).
+// ---------------------------------------------------------------------------------------------
+template <typename T>
+inline int64_t beaver_ws_words(int64_t M, int64_t K, int64_t N) {
+    return 2 * M * K + 2 * K * N + 2 * M * N;
+}
+
+template <typename T>
+psml_status beaver_matmul(const T *const A[2], const T *const B[2], const T *const U[2],
+                          const T *const V[2], const T *const Z[2], int64_t M, int64_t K,
+                          int64_t N, int flags, int trunc, T *const C[2], T *ws, int64_t ws_words,
+                          cudaStream_t s, int sm_count, T *const traceE[2] = nullptr,
+                          T *const traceF[2] = nullptr) {
+    T *mE0 = ws, *mE1 = ws + M * K, *mF0 = ws + 2 * M * K, *mF1 = mF0 + K * N;
+    T *partial = mF1 + K * N;
+    const int tA = (flags & PSML_TRANS_A) ? 1 : 0, tB = (flags & PSML_TRANS_B) ? 1 : 0;
+    MaskJobs<T> jobs;
+    jobs.j[0] = {A[0], U[0], mE0, M, K, tA};
+    jobs.j[1] = {A[1], U[1], mE1, M, K, tA};
+    jobs.j[2] = {B[0], V[0], mF0, K, N, tB};
+    jobs.j[3] = {B[1], V[1], mF1, K, N, tB};
+    jobs.count = 4;
+    const int64_t maxt = std::max(((M + 31) / 32) * ((K + 31) / 32), ((K + 31) / 32) * ((N + 31) / 32));
+    mask_kernel<T><<<dim3((unsigned)std::min<int64_t>(maxt, 148 * 8), 1, 4), dim3(32, 8), 0, s>>>(jobs);
+    PSML_LAUNCH_CHECK();
+    BeaverOps<T> ops;
+    ops.mE0 = mE0; ops.mE1 = mE1; ops.mF0 = mF0; ops.mF1 = mF1;
+    for (int p = 0; p < 2; ++p) {
+        ops.U[p] = U[p]; ops.V[p] = V[p]; ops.Z[p] = Z[p]; ops.A[p] = A[p]; ops.B[p] = B[p]; ops.C[p] = C[p];
+    }
+    ops.M = M; ops.N = N; ops.K = K; ops.Kext = 2 * K;
+    ops.form = (flags & PSML_PAPER_FORM) ? 1 : 0;
+    ops.transA = tA; ops.transB = tB; ops.trunc = trunc;
+    PSML_TRY((launch_ring_gemm<T, BeaverOps<T>>(ops, partial, ws_words - (partial - ws), s, sm_count)));
+    if (traceE) {
+        for (int p = 0; p < 2; ++p)
+            if (traceE[p]) PSML_CUDA_TRY(cudaMemcpyAsync(traceE[p], p ? mE1 : mE0, sizeof(T) * M * K, cudaMemcpyDeviceToDevice, s));
+    }
+    if (traceF) {
+        for (int p = 0; p < 2; ++p)
+            if (traceF[p]) PSML_CUDA_TRY(cudaMemcpyAsync(traceF[p], p ? mF1 : mF0, sizeof(T) * K * N, cudaMemcpyDeviceToDevice, s));
+    }
+    return PSML_OK;
+}
+
+// ---------------------------------------------------------------------------------------------
+// Convolution Beaver product (im2col ring GEMM, mask on the raw input; R17)
+// transposed = 0: C = im2col(X) . Wc         M = B*OH*OW, K = C*k*k,  N = Cout
+// transposed = 1: C = im2col(X)^T . D        M = C*k*k,   K = B*OH*OW, N = Cout
+// ws: 2*nin (raw-input messages) + 2*K*N (F messages) + 2*M*N (split-K)
+// ---------------------------------------------------------------------------------------------
+template <typename T>
+psml_status conv_beaver(const T *const X[2], const T *const Bm[2], const T *const UX[2],
+                        const T *const V[2], const T *const Z[2], int64_t batch, ConvGeom g,
+                        int transposed, int64_t N, int trunc, T *const C[2], T *ws, int64_t ws_words,
+                        cudaStream_t s, int sm_count) {
+    const int64_t nin = batch * g.C * g.H * g.W;
+    const int64_t rows = batch * g.OH * g.OW, kk = (int64_t)g.C * g.k * g.k;
+    const int64_t M = transposed ? kk : rows, K = transposed ? rows : kk;
+    T *mE0 = ws, *mE1 = ws + nin, *mF0 = ws + 2 * nin, *mF1 = mF0 + K * N, *partial = mF1 + K * N;
+    MaskJobs<T> jobs;
+    jobs.j[0] = {X[0], UX[0], mE0, batch, (int64_t)g.C * g.H * g.W, 0};
+    jobs.j[1] = {X[1], UX[1], mE1, batch, (int64_t)g.C * g.H * g.W, 0};
+    jobs.j[2] = {Bm[0], V[0], mF0, K, N, 0};
+    jobs.j[3] = {Bm[1], V[1], mF1, K, N, 0};
+    jobs.count = 4;
+    const int64_t maxt = std::max(((batch + 31) / 32) * (((int64_t)g.C * g.H * g.W + 31) / 32), ((K + 31) / 32) * ((N + 31) / 32));
+    mask_kernel<T><<<dim3((unsigned)std::min<int64_t>(maxt, 148 * 8), 1, 4), dim3(32, 8), 0, s>>>(jobs);
+    PSML_LAUNCH_CHECK();
+    ConvBeaverOps<T> ops;
+    ops.mE0 = mE0; ops.mE1 = mE1; ops.mF0 = mF0; ops.mF1 = mF1;
+    for (int p = 0; p < 2; ++p) { ops.UX[p] = UX[p]; ops.V[p] = V[p]; ops.Z[p] = Z[p]; ops.C[p] = C[p]; }
+    ops.g = g; ops.M = M; ops.N = N; ops.K = K; ops.Kext = 2 * K; ops.transposed = transposed; ops.trunc = trunc;
+    return launch_ring_gemm<T, ConvBeaverOps<T>>(ops, partial, ws_words - (partial - ws), s, sm_count);
+}
+
+template <typename T>
+inline int64_t conv_ws_words(int64_t batch, ConvGeom g, int transposed, int64_t N) {
+    const int64_t nin = batch * g.C * g.H * g.W;
+    const int64_t rows = batch * g.OH * g.OW, kk = (int64_t)g.C * g.k * g.k;
+    const int64_t M = transposed ? kk : rows, K = transposed ? rows : kk;
+    return 2 * nin + 2 * K * N + 2 * M * N;
+}
+
+// ---------------------------------------------------------------------------------------------
+// Hadamard (2 rounds).  ws: 4 n words.
+// ---------------------------------------------------------------------------------------------
+template <typename T>
+psml_status beaver_hadamard(const T *const A[2], const T *const B[2], const T *const U[2],
+                            const T *const V[2], const T *const Z[2], int64_t n, int trunc,
+                            T *const C[2], T *ws, cudaStream_t s) {
+    Pair<T> mE{{ws, ws + n}}, mF{{ws + 2 * n, ws + 3 * n}};
+    CPair<T> a{{A[0], A[1]}}, b{{B[0], B[1]}}, u{{U[0], U[1]}}, v{{V[0], V[1]}}, z{{Z[0], Z[1]}};
+    hadamard_mask_kernel<T><<<ew_grid(n), EW_THREADS, 0, s>>>(a, b, u, v, n, mE, mF);
+    PSML_LAUNCH_CHECK();
+    CPair<T> ce{{mE.p[0], mE.p[1]}}, cf{{mF.p[0], mF.p[1]}};
+    hadamard_open_kernel<T><<<ew_grid(n), EW_THREADS, 0, s>>>(ce, cf, u, v, z, n, trunc, Pair<T>{{C[0], C[1]}});
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
+// ---------------------------------------------------------------------------------------------
+// MSB chain and the activations built on it.  ws: 6 n words per party (G, P, 4 msg) = 12 n.
+// what: 0 = msb only (msbA), 1 = ReLU (y = x . drelu), 2 = Eq. 9 (x given as z of n/2; y of n/2,
+//       optional delta = y - Ysub).
+// ---------------------------------------------------------------------------------------------
+template <typename T>
+inline int64_t msb_ws_words(int64_t n) { return 12 * n; }
+
+template <typename T>
+psml_status msb_chain(const T *const x[2], int64_t n, const T *const mat[2], int mode, T half,
+                      int what, T *const msbA[2], T *const msbB[2], T *const drelu[2],
+                      const T *const U[2], const T *const V[2], const T *const Z[2], T *const y[2],
+                      const T *const Ysub[2], T *const delta[2], T *ws, cudaStream_t s) {
+    const int l = 8 * (int)sizeof(T);
+    MsbArgs<T> a;
+    a.x = CPair<T>{{x[0], x[1]}};
+    a.mat = CPair<T>{{mat[0], mat[1]}};
+    a.G = Pair<T>{{ws, ws + n}};
+    a.P = Pair<T>{{ws + 2 * n, ws + 3 * n}};
+    a.msg = Pair<T>{{ws + 4 * n, ws + 8 * n}};
+    a.n = n; a.mode = mode; a.half = half; a.L = ilog2_int(l); a.l = l;
+    const int g = ew_grid(n);
+    msb_round0_kernel<T><<<g, EW_THREADS, 0, s>>>(a);
+    PSML_LAUNCH_CHECK();
+    for (int j = 1; j <= a.L; ++j) {
+        msb_level_kernel<T><<<g, EW_THREADS, 0, s>>>(a, j);
+        PSML_LAUNCH_CHECK();
+    }
+    Pair<T> mb{{msbB ? msbB[0] : nullptr, msbB ? msbB[1] : nullptr}};
+    msb_final_kernel<T><<<g, EW_THREADS, 0, s>>>(a, mb);
+    PSML_LAUNCH_CHECK();
+    Pair<T> mE{{a.msg.p[0] + n, a.msg.p[1] + n}}, mF{{a.msg.p[0] + 2 * n, a.msg.p[1] + 2 * n}};
+    Pair<T> ma{{msbA ? msbA[0] : nullptr, msbA ? msbA[1] : nullptr}};
+    Pair<T> dr{{drelu ? drelu[0] : nullptr, drelu ? drelu[1] : nullptr}};
+    CPair<T> u{{U ? U[0] : nullptr, U ? U[1] : nullptr}}, v{{V ? V[0] : nullptr, V ? V[1] : nullptr}};
+    msb_b2a_kernel<T><<<g, EW_THREADS, 0, s>>>(a, ma, dr, u, v, mE, mF, what == 0 ? 0 : 1);
+    PSML_LAUNCH_CHECK();
+    if (what == 0) return PSML_OK;
+    CPair<T> ce{{mE.p[0], mE.p[1]}}, cf{{mF.p[0], mF.p[1]}}, z{{Z[0], Z[1]}};
+    if (what == 1) {
+        hadamard_open_kernel<T><<<g, EW_THREADS, 0, s>>>(ce, cf, u, v, z, n, 0, Pair<T>{{y[0], y[1]}});
+    } else {
+        const int64_t nh = n / 2;
+        Pair<T> yy{{y ? y[0] : nullptr, y ? y[1] : nullptr}};
+        CPair<T> ys{{Ysub ? Ysub[0] : nullptr, Ysub ? Ysub[1] : nullptr}};
+        Pair<T> dd{{delta ? delta[0] : nullptr, delta ? delta[1] : nullptr}};
+        eq9_open_kernel<T><<<ew_grid(nh), EW_THREADS, 0, s>>>(ce, cf, u, v, z, nh, yy, ys, dd);
+    }
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
+}  // namespace psml

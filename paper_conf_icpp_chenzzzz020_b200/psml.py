@@ -1,0 +1,416 @@
+"""Thin ctypes binding of libpsml.so (include/psml.h).  Argument marshalling only: every step of
+the hot path runs in the library's CUDA kernels.  PyTorch supplies device memory and streams.
+
+There is no CPU fallback: importing works anywhere (so the CPU test suite can check the
+exported symbols), but every compute call raises if the library or a CUDA device is missing.
+Function names follow the C ABI without the ``psml_`` prefix.
+"""
+import ctypes
+import os
+
+import torch
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(HERE, "libpsml.so")
+HEADER = os.path.join(os.path.dirname(HERE), "include", "psml.h")
+
+STATUS = {0: "PSML_OK", 1: "PSML_ERR_INVALID", 2: "PSML_ERR_SHAPE", 3: "PSML_ERR_ALIGN",
+          4: "PSML_ERR_UNSUPPORTED", 5: "PSML_ERR_CUDA", 6: "PSML_ERR_NOMEM", 7: "PSML_ERR_STATE"}
+TRANS_A, TRANS_B, PAPER_FORM = 1, 2, 4
+LINREG, LOGREG, MLP, CNN = 0, 1, 2, 3
+
+vp, i32, i64, u32, u64 = (ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64, ctypes.c_uint32,
+                          ctypes.c_uint64)
+P2 = vp * 2
+
+
+class PsmlError(RuntimeError):
+    def __init__(self, fn, status, msg):
+        super().__init__(f"{fn}: {STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class Ring(ctypes.Structure):
+    _fields_ = [("l", i32), ("frac_bits", i32)]
+
+
+class Trace(ctypes.Structure):
+    _fields_ = [("E", vp * 2), ("E_open", vp), ("F", vp * 2), ("F_open", vp)]
+
+
+class ModelDesc(ctypes.Structure):
+    _fields_ = [("kind", i32), ("n_layers", i32), ("dims", i64 * 8), ("batch", i32),
+                ("lr_shift", i32), ("master_frac_bits", i32), ("dealer_seed", u64),
+                ("pair_id", u32), ("cnn_c", i32), ("cnn_h", i32), ("cnn_w", i32), ("cnn_k", i32),
+                ("cnn_cout", i32), ("cnn_hidden", i32), ("cnn_classes", i32)]
+
+
+# name -> (restype, argtypes); mirrors include/psml.h
+_SIGS = {
+    "psml_abi_version": (i32, []),
+    "psml_last_error": (ctypes.c_char_p, []),
+    "psml_device_info": (i32, [vp, vp, vp]),
+    "psml_kernel_launch_count": (u64, []),
+    "psml_ctx_create": (i32, [Ring, i32, vp]),
+    "psml_ctx_destroy": (i32, [vp]),
+    "psml_prg_fill": (i32, [Ring, u64, u32, u64, u64, i64, vp, vp]),
+    "psml_encode": (i32, [Ring, vp, i64, vp, vp]),
+    "psml_decode": (i32, [Ring, vp, i64, vp, vp]),
+    "psml_share": (i32, [Ring, u64, u64, vp, i64, vp, vp, vp]),
+    "psml_reconstruct": (i32, [Ring, vp, vp, i64, vp, vp]),
+    "psml_triplet_gen": (i32, [vp, u64, u64, i64, i64, i64, P2, P2, P2, vp]),
+    "psml_hadamard_triplet_gen": (i32, [Ring, u64, u64, i64, P2, P2, P2, vp]),
+    "psml_msb_material_words": (i64, [Ring, i64]),
+    "psml_msb_dealer": (i32, [Ring, u64, u64, i64, P2, vp]),
+    "psml_secure_matmul": (i32, [vp, P2, P2, P2, P2, P2, i64, i64, i64, i32, i32, P2, vp, vp]),
+    "psml_secure_hadamard": (i32, [vp, P2, P2, P2, P2, P2, i64, i32, P2, vp]),
+    "psml_truncate": (i32, [Ring, i32, vp, i64, i32, vp]),
+    "psml_secure_msb": (i32, [vp, P2, i64, P2, P2, vp, vp]),
+    "psml_secure_relu": (i32, [vp, P2, i64, P2, P2, P2, P2, P2, vp, vp]),
+    "psml_secure_eq9": (i32, [vp, P2, i64, P2, P2, P2, P2, P2, vp]),
+    "psml_ring_gemm": (i32, [vp, vp, vp, i64, i64, i64, vp, vp]),
+    "psml_delta_encode": (i32, [vp, vp, vp, i64, i64, vp, vp, vp, vp, vp, vp, vp]),
+    "psml_delta_apply": (i32, [vp, i64, i64, i32, vp, vp, vp, vp, vp, vp]),
+    "psml_model_create": (i32, [vp, ctypes.POINTER(ModelDesc), vp]),
+    "psml_model_destroy": (i32, [vp]),
+    "psml_model_layer_shape": (i32, [vp, i32, vp, vp]),
+    "psml_model_set_master": (i32, [vp, i32, P2, vp]),
+    "psml_model_get_master": (i32, [vp, i32, P2, vp]),
+    "psml_model_deal": (i32, [vp, u32, i32, vp]),
+    "psml_secure_train_step": (i32, [vp, P2, P2, u32, vp]),
+    "psml_train_forward_backward": (i32, [vp, P2, P2, u32, vp]),
+    "psml_model_grads": (i32, [vp, vp, vp]),
+    "psml_train_apply_update": (i32, [vp, i32, vp]),
+    "psml_secure_infer": (i32, [vp, P2, u32, P2, vp]),
+}
+EXPORTS = tuple(_SIGS)
+
+_lib = None
+
+
+def lib():
+    """Load libpsml.so (build it first with paper_conf_icpp_chenzzzz020_b200.build)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise PsmlError("load", 4, f"{LIB_PATH} missing: run `python -m "
+                            "paper_conf_icpp_chenzzzz020_b200.build` (no CPU fallback exists)")
+        L = ctypes.CDLL(LIB_PATH)
+        for name, (res, args) in _SIGS.items():
+            f = getattr(L, name)
+            f.restype = res
+            f.argtypes = args
+        _lib = L
+    return _lib
+
+
+def _call(name, *args):
+    st = getattr(lib(), name)(*args)
+    if st != 0:
+        raise PsmlError(name, st, lib().psml_last_error().decode(errors="replace"))
+
+
+# ---------------------------------------------------------------------------------------------
+# marshalling helpers
+# ---------------------------------------------------------------------------------------------
+def dtype_of(l):
+    return torch.uint64 if l == 64 else torch.uint32
+
+
+def _ptr(t):
+    if t is None:
+        return None
+    if not t.is_cuda:
+        raise PsmlError("marshal", 1, "tensor must be on a CUDA device")
+    if not t.is_contiguous():
+        raise PsmlError("marshal", 1, "tensor must be contiguous")
+    return ctypes.c_void_p(t.data_ptr())
+
+
+def _pair(ts):
+    if ts is None:
+        return None
+    return P2(*(None if t is None else t.data_ptr() for t in ts))
+
+
+def _stream(stream=None):
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+def empty(n, l, like_shape=None):
+    shape = like_shape if like_shape is not None else (n,)
+    return torch.empty(shape, dtype=dtype_of(l), device="cuda")
+
+
+def empty_pair(shape, l):
+    return (torch.empty(shape, dtype=dtype_of(l), device="cuda"),
+            torch.empty(shape, dtype=dtype_of(l), device="cuda"))
+
+
+def tag(s):
+    b = (s.encode() if isinstance(s, str) else bytes(s)) + b"\0\0\0\0"
+    return int.from_bytes(b[:4], "little")
+
+
+# ---------------------------------------------------------------------------------------------
+# library / device
+# ---------------------------------------------------------------------------------------------
+def abi_version():
+    return lib().psml_abi_version()
+
+
+def kernel_launch_count():
+    return lib().psml_kernel_launch_count()
+
+
+def device_info():
+    a, b, c = i32(), i32(), i32()
+    _call("psml_device_info", ctypes.byref(a), ctypes.byref(b), ctypes.byref(c))
+    return a.value, b.value, c.value
+
+
+class Ctx:
+    """psml_ctx: one per GPU and host thread.  backend: 0 auto, 1 CUDA-core, 2 tcgen05."""
+
+    def __init__(self, l=64, frac_bits=13, backend=0):
+        self.ring = Ring(l, frac_bits)
+        self.l = l
+        h = vp()
+        _call("psml_ctx_create", self.ring, backend, ctypes.byref(h))
+        self.handle = h
+
+    def close(self):
+        if self.handle:
+            lib().psml_ctx_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+# ---------------------------------------------------------------------------------------------
+# client / dealer
+# ---------------------------------------------------------------------------------------------
+def prg_fill(ring, seed, tag_value, call_id, n, offset=0, out=None, stream=None):
+    out = out if out is not None else empty(n, ring.l)
+    _call("psml_prg_fill", ring, seed, tag_value, call_id, offset, n, _ptr(out), _stream(stream))
+    return out
+
+
+def encode(ring, x, stream=None):
+    x = x.to(dtype=torch.float64, device="cuda").contiguous()
+    v = torch.empty(x.shape, dtype=dtype_of(ring.l), device="cuda")
+    _call("psml_encode", ring, _ptr(x), x.numel(), _ptr(v), _stream(stream))
+    return v
+
+
+def decode(ring, v, stream=None):
+    x = torch.empty(v.shape, dtype=torch.float64, device="cuda")
+    _call("psml_decode", ring, _ptr(v), v.numel(), _ptr(x), _stream(stream))
+    return x
+
+
+def share(ring, seed, stream_id, x, out=None, stream=None):
+    x0, x1 = out if out is not None else empty_pair(x.shape, ring.l)
+    _call("psml_share", ring, seed, stream_id, _ptr(x), x.numel(), _ptr(x0), _ptr(x1),
+          _stream(stream))
+    return x0, x1
+
+
+def reconstruct(ring, x0, x1, stream=None):
+    x = torch.empty_like(x0)
+    _call("psml_reconstruct", ring, _ptr(x0), _ptr(x1), x0.numel(), _ptr(x), _stream(stream))
+    return x
+
+
+def triplet_gen(ctx, seed, call_id, M, K, N, stream=None):
+    U, V, Z = empty_pair((M, K), ctx.l), empty_pair((K, N), ctx.l), empty_pair((M, N), ctx.l)
+    _call("psml_triplet_gen", ctx.handle, seed, call_id, M, K, N, _pair(U), _pair(V), _pair(Z),
+          _stream(stream))
+    return U, V, Z
+
+
+def hadamard_triplet_gen(ring, seed, call_id, n, stream=None):
+    U, V, Z = empty_pair(n, ring.l), empty_pair(n, ring.l), empty_pair(n, ring.l)
+    _call("psml_hadamard_triplet_gen", ring, seed, call_id, n, _pair(U), _pair(V), _pair(Z),
+          _stream(stream))
+    return U, V, Z
+
+
+def msb_material_words(ring, n):
+    return lib().psml_msb_material_words(ring, n)
+
+
+def msb_dealer(ring, seed, call_id, n, stream=None):
+    mat = empty_pair(msb_material_words(ring, n), ring.l)
+    _call("psml_msb_dealer", ring, seed, call_id, n, _pair(mat), _stream(stream))
+    return mat
+
+
+# ---------------------------------------------------------------------------------------------
+# server side
+# ---------------------------------------------------------------------------------------------
+def secure_matmul(ctx, A, B, U, V, Z, M, K, N, flags=0, trunc=0, out=None, trace=False,
+                  stream=None):
+    C = out if out is not None else empty_pair((M, N), ctx.l)
+    tr = None
+    tr_t = None
+    if trace:
+        tr_t = dict(E0=empty(0, ctx.l, (M, K)), E1=empty(0, ctx.l, (M, K)), E=empty(0, ctx.l, (M, K)),
+                    F0=empty(0, ctx.l, (K, N)), F1=empty(0, ctx.l, (K, N)), F=empty(0, ctx.l, (K, N)))
+        tr = Trace(P2(tr_t["E0"].data_ptr(), tr_t["E1"].data_ptr()), tr_t["E"].data_ptr(),
+                   P2(tr_t["F0"].data_ptr(), tr_t["F1"].data_ptr()), tr_t["F"].data_ptr())
+    _call("psml_secure_matmul", ctx.handle, _pair(A), _pair(B), _pair(U), _pair(V), _pair(Z),
+          M, K, N, flags, trunc, _pair(C), ctypes.byref(tr) if tr is not None else None,
+          _stream(stream))
+    return (C, tr_t) if trace else C
+
+
+def secure_hadamard(ctx, A, B, U, V, Z, trunc=0, out=None, stream=None):
+    n = A[0].numel()
+    C = out if out is not None else empty_pair(A[0].shape, ctx.l)
+    _call("psml_secure_hadamard", ctx.handle, _pair(A), _pair(B), _pair(U), _pair(V), _pair(Z), n,
+          trunc, _pair(C), _stream(stream))
+    return C
+
+
+def truncate(ring, party, x, bits, stream=None):
+    _call("psml_truncate", ring, party, _ptr(x), x.numel(), bits, _stream(stream))
+    return x
+
+
+def secure_msb(ctx, x, mat, want_bool=False, stream=None):
+    n = x[0].numel()
+    a = empty_pair(x[0].shape, ctx.l)
+    b = empty_pair(x[0].shape, ctx.l) if want_bool else None
+    _call("psml_secure_msb", ctx.handle, _pair(x), n, _pair(mat), _pair(a), _pair(b),
+          _stream(stream))
+    return (a, b) if want_bool else a
+
+
+def secure_relu(ctx, x, mat, U, V, Z, stream=None):
+    n = x[0].numel()
+    y, d = empty_pair(x[0].shape, ctx.l), empty_pair(x[0].shape, ctx.l)
+    _call("psml_secure_relu", ctx.handle, _pair(x), n, _pair(mat), _pair(U), _pair(V), _pair(Z),
+          _pair(y), _pair(d), _stream(stream))
+    return y, d
+
+
+def secure_eq9(ctx, x, mat, U, V, Z, stream=None):
+    n = x[0].numel()
+    y = empty_pair(x[0].shape, ctx.l)
+    _call("psml_secure_eq9", ctx.handle, _pair(x), n, _pair(mat), _pair(U), _pair(V), _pair(Z),
+          _pair(y), _stream(stream))
+    return y
+
+
+def ring_gemm(ctx, A, B, out=None, stream=None):
+    M, K = A.shape
+    N = B.shape[1]
+    C = out if out is not None else empty(0, ctx.l, (M, N))
+    _call("psml_ring_gemm", ctx.handle, _ptr(A), _ptr(B), M, K, N, _ptr(C), _stream(stream))
+    return C
+
+
+def delta_encode(ctx, cur, prev, stream=None):
+    rows, cols = cur.shape
+    row_ptr = torch.empty(rows + 1, dtype=torch.int32, device="cuda")
+    col_idx = torch.empty(rows * cols, dtype=torch.int32, device="cuda")
+    vals = empty(rows * cols, ctx.l)
+    dense = empty(0, ctx.l, (rows, cols))
+    nnz, is_csr = i64(), i32()
+    _call("psml_delta_encode", ctx.handle, _ptr(cur), _ptr(prev), rows, cols, _ptr(row_ptr),
+          _ptr(col_idx), _ptr(vals), _ptr(dense), ctypes.byref(nnz), ctypes.byref(is_csr),
+          _stream(stream))
+    if is_csr.value:
+        return dict(is_csr=True, nnz=nnz.value, row_ptr=row_ptr, col_idx=col_idx[:nnz.value],
+                    vals=vals[:nnz.value])
+    return dict(is_csr=False, nnz=nnz.value, dense=dense)
+
+
+def delta_apply(ctx, target, enc, stream=None):
+    rows, cols = target.shape
+    if enc["is_csr"]:
+        _call("psml_delta_apply", ctx.handle, rows, cols, 1, _ptr(enc["row_ptr"]),
+              _ptr(enc["col_idx"]), _ptr(enc["vals"]) if enc["nnz"] else None, None, _ptr(target),
+              _stream(stream))
+    else:
+        _call("psml_delta_apply", ctx.handle, rows, cols, 0, None, None, None, _ptr(enc["dense"]),
+              _ptr(target), _stream(stream))
+    return target
+
+
+# ---------------------------------------------------------------------------------------------
+# models
+# ---------------------------------------------------------------------------------------------
+class Model:
+    """psml_model: weight shares, dealer pool and workspaces of one secure model."""
+
+    def __init__(self, ctx, kind, dims=None, batch=128, lr_shift=14, master_frac_bits=27,
+                 dealer_seed=0x50534D4C + 2, pair_id=0, cnn=(3, 32, 32, 5, 16, 64, 10)):
+        d = ModelDesc()
+        d.kind = kind
+        dims = list(dims or ([784, 1] if kind in (LINREG, LOGREG) else [784, 128, 128, 10]))
+        d.n_layers = 3 if kind == CNN else len(dims) - 1
+        for i, v in enumerate(dims[:8]):
+            d.dims[i] = v
+        d.batch, d.lr_shift, d.master_frac_bits = batch, lr_shift, master_frac_bits
+        d.dealer_seed, d.pair_id = dealer_seed, pair_id
+        (d.cnn_c, d.cnn_h, d.cnn_w, d.cnn_k, d.cnn_cout, d.cnn_hidden, d.cnn_classes) = cnn
+        self.ctx, self.desc, self.kind = ctx, d, kind
+        h = vp()
+        _call("psml_model_create", ctx.handle, ctypes.byref(d), ctypes.byref(h))
+        self.handle = h
+        self.n_layers = d.n_layers
+
+    def layer_shape(self, layer):
+        r, c = i64(), i64()
+        _call("psml_model_layer_shape", self.handle, layer, ctypes.byref(r), ctypes.byref(c))
+        return r.value, c.value
+
+    def set_master(self, layer, Wm, stream=None):
+        _call("psml_model_set_master", self.handle, layer, _pair(Wm), _stream(stream))
+
+    def get_master(self, layer, stream=None):
+        W = empty_pair(self.layer_shape(layer), self.ctx.l)
+        _call("psml_model_get_master", self.handle, layer, _pair(W), _stream(stream))
+        return W
+
+    def deal(self, step, infer_only=False, stream=None):
+        _call("psml_model_deal", self.handle, step, 1 if infer_only else 0, _stream(stream))
+
+    def train_step(self, X, Y, step, stream=None):
+        _call("psml_secure_train_step", self.handle, _pair(X), _pair(Y), step, _stream(stream))
+
+    def forward_backward(self, X, Y, step, stream=None):
+        _call("psml_train_forward_backward", self.handle, _pair(X), _pair(Y), step,
+              _stream(stream))
+
+    def grads(self):
+        """(pointer, words per party) of the model-owned [2][P] gradient buffer."""
+        p, n = vp(), i64()
+        _call("psml_model_grads", self.handle, ctypes.byref(p), ctypes.byref(n))
+        return p.value, n.value
+
+    def apply_update(self, extra_shift=0, stream=None):
+        _call("psml_train_apply_update", self.handle, extra_shift, _stream(stream))
+
+    def infer(self, X, step, out_shape, stream=None):
+        Y = empty_pair(out_shape, self.ctx.l)
+        _call("psml_secure_infer", self.handle, _pair(X), step, _pair(Y), _stream(stream))
+        return Y
+
+    def close(self):
+        if self.handle:
+            lib().psml_model_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

@@ -1,0 +1,122 @@
+"""Secure training / inference driver over the C ABI (the API a user calls).
+
+Roles (Fig. 1b, L55-L65; Fig. 3):
+  client  encodes plaintext (fixed point, f = 13) and splits it into two additive shares
+          (psml_encode + psml_share on the GPU, streams keyed by the call-id layout below);
+  dealer  generates the step's triplets / MSB material (psml_model_deal) -- the offline phase;
+  servers run the online step on the shares (psml_secure_train_step), both parties co-resident.
+
+Call-id layout (R11; part of the bit-exact contract with the oracle):
+  pair[63:56] | step[55:24] | layer[23:16] | op[15:8] | slot[7:0]
+  op 7 = share; slot 0 = X, 1 = Y, 2 = initial master weight (step = 0xFFFFFFFF).
+Data parallelism: one co-resident pair per GPU, each on its own rows;
+the untruncated weight-gradient shares are summed across pairs with an all-reduce (uint64 ring
+addition = int64 two's-complement addition), then every pair applies the same update.
+"""
+import math
+
+import torch
+
+from . import psml
+
+DATA_SEED = 0x50534D4C
+SHARE_SEED = DATA_SEED + 1
+DEALER_SEED = DATA_SEED + 2
+OP_SHARE = 7
+INIT_STEP = 0xFFFFFFFF
+KINDS = {"linreg": psml.LINREG, "logreg": psml.LOGREG, "mlp": psml.MLP, "cnn": psml.CNN}
+
+
+def call_id(pair, step, layer, op, slot=0):
+    return ((pair & 0xFF) << 56) | ((step & 0xFFFFFFFF) << 24) | ((layer & 0xFF) << 16) \
+        | ((op & 0xFF) << 8) | (slot & 0xFF)
+
+
+class SecureTrainer:
+    """One co-resident party pair on the current GPU, training `task` with batch `batch`."""
+
+    def __init__(self, task, W_init, batch=128, pair_id=0, dims=None, backend=0,
+                 frac_bits=13, master_frac_bits=27, lr_shift=14):
+        self.task = task
+        self.ctx = psml.Ctx(l=64, frac_bits=frac_bits, backend=backend)
+        self.ring = self.ctx.ring
+        self.master_ring = psml.Ring(64, master_frac_bits)
+        self.pair_id = pair_id
+        self.batch = batch
+        self.model = psml.Model(self.ctx, KINDS[task], dims=dims, batch=batch, lr_shift=lr_shift,
+                                master_frac_bits=master_frac_bits, dealer_seed=DEALER_SEED,
+                                pair_id=pair_id)
+        for layer, W in enumerate(W_init):
+            w = psml.encode(self.master_ring, torch.as_tensor(W, dtype=torch.float64))
+            Wm = psml.share(self.ring, SHARE_SEED, call_id(0, INIT_STEP, layer, OP_SHARE, 2), w)
+            self.model.set_master(layer, Wm)
+        self.out_dim = self.model.layer_shape(self.model.n_layers - 1)[1]
+
+    # --- client side -----------------------------------------------------------------------
+    def share_batch(self, X, Y, step):
+        """Encode + share one minibatch on the GPU (X, Y: float64 tensors, host or device)."""
+        x = psml.encode(self.ring, torch.as_tensor(X, dtype=torch.float64))
+        y = psml.encode(self.ring, torch.as_tensor(Y, dtype=torch.float64))
+        Xs = psml.share(self.ring, SHARE_SEED, call_id(self.pair_id, step, 0, OP_SHARE, 0), x)
+        Ys = psml.share(self.ring, SHARE_SEED, call_id(self.pair_id, step, 0, OP_SHARE, 1), y)
+        return Xs, Ys
+
+    # --- steps --------------------------------------------------------------------------------
+    def deal(self, step, infer_only=False):
+        self.model.deal(step, infer_only=infer_only)
+
+    def step_shares(self, Xs, Ys, step, deal=True):
+        if deal:
+            self.model.deal(step)
+        self.model.train_step(Xs, Ys, step)
+
+    def step(self, X, Y, step):
+        Xs, Ys = self.share_batch(X, Y, step)
+        self.step_shares(Xs, Ys, step)
+
+    def step_dp(self, Xs, Ys, step, group=None, deal=True):
+        """Data-parallel step: local forward/backward, all-reduce of gradient shares, update."""
+        import torch.distributed as dist
+        if deal:
+            self.model.deal(step)
+        self.model.forward_backward(Xs, Ys, step)
+        world = dist.get_world_size(group) if dist.is_initialized() else 1
+        if world > 1:
+            g = self.grad_tensor()
+            dist.all_reduce(g, op=dist.ReduceOp.SUM, group=group)
+        extra = int(round(math.log2(world)))
+        if (1 << extra) != world:
+            raise ValueError("data-parallel pair count must be a power of two (R16)")
+        self.model.apply_update(extra_shift=extra)
+
+    def grad_tensor(self):
+        """int64 view of the model-owned [2][P] gradient buffer (for the all-reduce)."""
+        ptr, words = self.model.grads()
+        return _wrap_device_ptr(ptr, 2 * words)
+
+    def infer_shares(self, Xs, step):
+        self.model.deal(step, infer_only=True)
+        return self.model.infer(Xs, step, (Xs[0].shape[0], self.out_dim))
+
+    # --- decode (client side, test/report only) ---------------------------------------------------
+    def master_weights(self):
+        out = []
+        for layer in range(self.model.n_layers):
+            W0, W1 = self.model.get_master(layer)
+            out.append(psml.decode(self.master_ring, psml.reconstruct(self.ring, W0, W1)))
+        return out
+
+    def master_shares(self, layer):
+        return self.model.get_master(layer)
+
+    def close(self):
+        self.model.close()
+        self.ctx.close()
+
+
+def _wrap_device_ptr(ptr, numel):
+    """A torch int64 tensor aliasing `numel` words of library-owned device memory."""
+    class _Holder:
+        __cuda_array_interface__ = {"shape": (numel,), "typestr": "<i8", "data": (ptr, False),
+                                    "version": 3, "strides": None}
+    return torch.as_tensor(_Holder(), device="cuda")

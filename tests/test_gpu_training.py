@@ -1,0 +1,79 @@
+"""GPU secure training / inference vs the oracle (bit-exact) and vs fp64 (BASELINE 2^-12 pin).
+
+Bit-exact: after each step, both parties' master-weight shares equal the oracle's simulation of
+the same protocol (oracle/protocol.py) on the same seeded inputs.  Accuracy: after one full
+epoch, the decoded master weights are within 2^-12 of plaintext fp64 SGD (oracle/plain.py).
+"""
+import numpy as np
+import pytest
+import torch
+
+import synth
+from oracle import plain
+from oracle import protocol as OP
+from tests.util import to_np
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def T():
+    from paper_conf_icpp_chenzzzz020_b200 import build, train
+    build.build()
+    return train
+
+
+def _compare_shares(tr, om):
+    for layer in range(len(om.Wm)):
+        g0, g1 = tr.master_shares(layer)
+        assert np.array_equal(to_np(g0).reshape(om.Wm[layer][0].shape), om.Wm[layer][0]), layer
+        assert np.array_equal(to_np(g1).reshape(om.Wm[layer][1].shape), om.Wm[layer][1]), layer
+
+
+@pytest.mark.parametrize("task,steps", [("linreg", 3), ("logreg", 3), ("mlp", 3), ("cnn", 1)])
+def test_training_bitexact_vs_oracle(T, task, steps):
+    Wi = synth.init_weights(task)
+    tr = T.SecureTrainer(task, Wi, backend=1)
+    om = OP.Model(task, Wi)
+    _compare_shares(tr, om)
+    for s in range(steps):
+        X, Y = synth.batch(task, s)
+        tr.step(torch.from_numpy(X), torch.from_numpy(Y), s)
+        OP.train_step(om, X, Y, s)
+        torch.cuda.synchronize()
+        _compare_shares(tr, om)
+    tr.close()
+
+
+@pytest.mark.parametrize("task", ["mlp", "logreg"])
+def test_inference_bitexact_vs_oracle(T, task):
+    Wi = synth.init_weights(task)
+    tr = T.SecureTrainer(task, Wi, backend=1)
+    om = OP.Model(task, Wi)
+    X, Y = synth.batch(task, 11)
+    Xs_g, _ = tr.share_batch(torch.from_numpy(X), torch.from_numpy(Y), 11)
+    Xs_o, _ = OP.share_batch(X, Y, 11)
+    yg = tr.infer_shares(Xs_g, 500)
+    yo = OP.infer(om, Xs_o, 500)
+    assert np.array_equal(to_np(yg[0]).reshape(yo[0].shape), yo[0])
+    assert np.array_equal(to_np(yg[1]).reshape(yo[1].shape), yo[1])
+    tr.close()
+
+
+@pytest.mark.parametrize("task,tol_log2", [("linreg", -12), ("logreg", -12), ("mlp", -12)])
+def test_one_epoch_within_2pow_minus12_of_fp64(T, task, tol_log2):
+    """BASELINE north_star: decoded weights within 2^-12 of plaintext fp64 after one epoch
+    (60000 MNIST-shaped rows, batch 128, 468 steps, R13-R15)."""
+    Wi = synth.init_weights(task)
+    tr = T.SecureTrainer(task, Wi, backend=0)
+    pm = plain.PlainModel(task, Wi)
+    steps = 60000 // 128
+    for s in range(steps):
+        X, Y = synth.batch(task, s)
+        tr.step(torch.from_numpy(X), torch.from_numpy(Y), s)
+        pm.step(X, Y)
+    got = [w.cpu().numpy() for w in tr.master_weights()]
+    err = max(np.abs(g.reshape(w.shape) - w).max() for g, w in zip(got, pm.W))
+    print(f"{task}: one-epoch max |w - w_fp64| = 2^{np.log2(err):.2f}")
+    assert err < 2.0 ** tol_log2
+    tr.close()
