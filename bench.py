@@ -35,8 +35,8 @@ INT8_DENSE_PEAK_TOPS = 4500.0   # B200 nominal dense INT8 (B200_PROFILING / NVID
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=50)
-    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-ring-gemm", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -190,9 +190,6 @@ def bench_ours(args):
     t_dev = max_over_ranks(t_dev, world)
 
     # online-only (dealer material generated before each step, outside the events)
-    def online(s):
-        pass
-    t_on = 0.0
     evs = []
     for i in range(K):
         s = W + K + i
@@ -218,9 +215,9 @@ def bench_ours(args):
         Y = Yh[i].to(dev, non_blocking=True)
         one_step(s, X, Y)
         # the step's result: both parties' prediction shares of this batch
-        ptr = tr.model  # noqa: F841
-        out_host[0].copy_(tr_out(tr)[0], non_blocking=True)
-        out_host[1].copy_(tr_out(tr)[1], non_blocking=True)
+        y0, y1 = tr.last_yhat()
+        out_host[0].view(-1).copy_(y0, non_blocking=True)
+        out_host[1].view(-1).copy_(y1, non_blocking=True)
     t_e2e = max_over_ranks(timed(e2e_step, K, 2 * (W + K)), world)
 
     samples = BATCH * K * world
@@ -239,12 +236,93 @@ def bench_ours(args):
         "gpu_launches": int(launches),
         "clocks": clk.summary(),
     }
+    # per-kernel-class time inside the same step (CUDA events on the launching stream)
+    classes = {}
+    base = 3 * (W + K)
+    for cls, name in ((psml.PROF_GEMM, "ring_gemm_cuda_core"), (psml.PROF_MSB, "msb_relu_eq9_rounds"),
+                      (psml.PROF_HAD, "hadamard_rounds"), (psml.PROF_DEALER, "dealer"),
+                      (psml.PROF_MASK, "beaver_mask")):
+        psml.prof_enable(cls)
+        psml.prof_read()
+        for i in range(K):
+            one_step(base + i, Xs[i % nb], Ys[i % nb])
+        ms, n, work = psml.prof_read()
+        psml.prof_enable(-1)
+        base += K
+        classes[name] = {"ms_per_step": ms / K, "share_of_step": (ms / K) / result["ms_per_step"],
+                         "launches_per_step": n / K, "work_per_launch": work / max(n, 1),
+                         "ms_per_launch": ms / max(n, 1)}
+    result["kernel_classes"] = classes
+    result["roofline"] = roofline(classes, result["clocks"])
     return result, tr, world, rank
 
 
-def tr_out(tr):
-    """Prediction shares of the last step (model-owned yhat) as torch views (for the D2H)."""
-    return tr.last_yhat()
+def measured_peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except (OSError, ValueError):
+        return {}
+
+
+def roofline(classes, clocks):
+    """Roofline of the dominant kernel class (largest share of the step), DESIGN.md Sec. 5."""
+    name = max(classes, key=lambda k: classes[k]["ms_per_step"])
+    c = classes[name]
+    sec = c["ms_per_launch"] / 1e3
+    mp = measured_peaks()
+    if name == "ring_gemm_cuda_core":
+        # ALU bound: a Z_2^64 multiply-add is 3 IMAD-pipe ops (IMAD.WIDE.U32 + 2 IMAD); B200:
+        # 148 SMs x 4 SMSPs x 16 lanes/clk at clocks.max.sm 1965 MHz (B300_MICROARCH rt=2)
+        peak = 148 * 64 / 3 * 1.965e9 / 1e12
+        ach = c["work_per_launch"] / sec / 1e12
+        return {"bound": "alu", "kernel": name, "achieved": ach, "peak": peak,
+                "unit": "T ring-MAC/s", "frac": ach / peak, "traffic": None,
+                "peak_source": "derived: 148 SM x 64 IMAD/clk / 3 IMAD per u64 MAC x 1965 MHz"}
+    peak = mp.get("hbm_gbs", 6650.0)
+    ach = c["work_per_launch"] / sec / 1e9
+    return {"bound": "hbm", "kernel": name, "achieved": ach, "peak": peak, "unit": "GB/s",
+            "frac": ach / peak, "traffic": None,
+            "peak_source": "measured" if "hbm_gbs" in mp else "fallback"}
+
+
+def ring_gemm_figure(n=4096, l=64, reps=5):
+    """BASELINE config 5 kernel: plain C = A B mod 2^l, n^3, timed with CUDA events."""
+    import torch
+    from paper_conf_icpp_chenzzzz020_b200 import psml
+    ctx = psml.Ctx(l=l)
+    ring = ctx.ring
+    A = psml.prg_fill(ring, 1, psml.tag("bA"), 0, n * n).view(n, n)
+    B = psml.prg_fill(ring, 1, psml.tag("bB"), 0, n * n).view(n, n)
+    C = psml.empty(0, l, (n, n))
+    psml.ring_gemm(ctx, A, B, out=C)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+    tot = 0.0
+    for _ in range(reps):
+        flush.zero_()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        psml.ring_gemm(ctx, A, B, out=C)
+        b.record()
+        torch.cuda.synchronize()
+        tot += a.elapsed_time(b)
+    ms = tot / reps
+    pairs = 36 if l == 64 else 10
+    useful = pairs * 2.0 * n ** 3
+    ctx.close()
+    return {"n": n, "l": l, "ms": ms, "useful_limb_tops": useful / (ms / 1e3) / 1e12,
+            "frac_of_int8_dense_peak_4500": useful / (ms / 1e3) / 1e12 / INT8_DENSE_PEAK_TOPS,
+            "ring_tmacs": n ** 3 / (ms / 1e3) / 1e12}
+
+
+def cpu_baseline(budget_s=12.0):
+    """The oracle as it stands on this host: whole secure MLP training steps (batch 128)."""
+    import oracle
+    oracle.build()
+    t1, cores = oracle_steps(1, base=10000)
+    n = max(2, min(60, int(budget_s / max(t1, 1e-3))))
+    t, cores = oracle_steps(n, base=10001)
+    return {"value": BATCH * n / t, "unit": "samples/s", "cores": cores, "kind": "oracle",
+            "sample": f"{n} full oracle secure MLP training steps (batch 128) on the host"}
 
 
 # ---------------------------------------------------------------------------------------------
@@ -291,6 +369,10 @@ def main():
             print(json.dumps(out), flush=True)
         return
     result, tr, world, rank = bench_ours(args)
+    if rank == 0 and world == 1 and not args.no_ring_gemm:
+        result["ring_gemm"] = [ring_gemm_figure(4096, 64), ring_gemm_figure(4096, 32)]
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        result["cpu_baseline"] = cpu_baseline()
     if rank == 0:
         print(json.dumps(result), flush=True)
 

@@ -72,6 +72,16 @@ psml_status psml_device_info(int32_t *sm_count, int32_t *cc_major, int32_t *cc_m
 /* Number of kernels this process has launched through the library (for bench accounting). */
 uint64_t psml_kernel_launch_count(void);
 
+/* Kernel-class timing for bench.py's roofline (off by default).  While enabled for class `cls`,
+ * every library launch of that class is bracketed by CUDA events on its own stream, and its
+ * algorithmic work is accumulated: ring GEMMs count ring multiply-adds (M*N*K' per party),
+ * the elementwise classes count algorithmic HBM bytes (each word read + written once).
+ * cls: 0 CUDA-core ring GEMM, 1 tcgen05 limb GEMM, 2 MSB/ReLU/Eq. 9 round kernels,
+ *      3 Hadamard rounds, 4 dealer PRG kernels, 5 Beaver masking, -1 = disable.
+ * psml_prof_read synchronizes the device, returns the totals and resets them. */
+psml_status psml_prof_enable(int32_t cls);
+psml_status psml_prof_read(double *total_ms, int64_t *launches, double *work);
+
 /* ------------------------------------------------------------------------------------------ */
 /* Context                                                                                     */
 /* ------------------------------------------------------------------------------------------ */
@@ -241,6 +251,8 @@ psml_status psml_secure_train_step(psml_model model, const void *const X[2],
 psml_status psml_train_forward_backward(psml_model model, const void *const X[2],
                                         const void *const Y[2], uint32_t step_id,
                                         psml_stream stream);
+/* Model-owned prediction shares of the last forward pass: yhat[i] is batch x d_L (device). */
+psml_status psml_model_output(psml_model model, void **yhat0, void **yhat1, int64_t *n);
 /* Contiguous gradient buffer: [party][all layers' rows*cols] words (device, model-owned). */
 psml_status psml_model_grads(psml_model model, void **grads, int64_t *words_per_party);
 /* W^m_i -= trunc_i(gradW_i, 26 + lr_shift - m + extra_shift); W_i = trunc_i(W^m_i, m - f).

@@ -34,6 +34,35 @@ extern std::atomic<uint64_t> g_launches;
             return ::psml::fail(PSML_ERR_CUDA, std::string("kernel launch: ") + cudaGetErrorString(_e)); \
     } while (0)
 
+// ---------------------------------------------------------------------------------------------
+// kernel-class profiling (psml_prof_enable / psml_prof_read): CUDA events around launches
+// ---------------------------------------------------------------------------------------------
+enum ProfClass { PROF_GEMM = 0, PROF_TC = 1, PROF_MSB = 2, PROF_HAD = 3, PROF_DEALER = 4, PROF_MASK = 5 };
+extern std::atomic<int> g_prof_cls;
+void prof_record(cudaEvent_t a, cudaEvent_t b, double work);
+cudaEvent_t prof_event();
+
+struct ProfScope {
+    bool on = false;
+    cudaEvent_t a = nullptr;
+    cudaStream_t s = nullptr;
+    double work = 0;
+    ProfScope(int cls, cudaStream_t st, double w) {
+        if (g_prof_cls.load(std::memory_order_relaxed) == cls) {
+            on = true; s = st; work = w;
+            a = prof_event();
+            cudaEventRecord(a, s);
+        }
+    }
+    ~ProfScope() {
+        if (on) {
+            cudaEvent_t b = prof_event();
+            cudaEventRecord(b, s);
+            prof_record(a, b, work);
+        }
+    }
+};
+
 #define PSML_TRY(expr)                          \
     do {                                        \
         psml_status _s = (expr);                \

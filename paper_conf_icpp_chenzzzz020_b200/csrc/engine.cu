@@ -4,6 +4,8 @@
 #include <cstring>
 #include <mutex>
 #include <string>
+#include <utility>
+#include <vector>
 
 #include "engine.h"
 
@@ -11,6 +13,30 @@ namespace psml {
 
 static thread_local std::string g_err;
 std::atomic<uint64_t> g_launches{0};
+
+std::atomic<int> g_prof_cls{-1};
+static std::mutex g_prof_mu;
+static std::vector<std::pair<cudaEvent_t, cudaEvent_t>> g_prof_pairs;
+static std::vector<cudaEvent_t> g_prof_pool;
+static double g_prof_work = 0;
+
+cudaEvent_t prof_event() {
+    std::lock_guard<std::mutex> lk(g_prof_mu);
+    if (!g_prof_pool.empty()) {
+        cudaEvent_t e = g_prof_pool.back();
+        g_prof_pool.pop_back();
+        return e;
+    }
+    cudaEvent_t e = nullptr;
+    cudaEventCreate(&e);
+    return e;
+}
+
+void prof_record(cudaEvent_t a, cudaEvent_t b, double work) {
+    std::lock_guard<std::mutex> lk(g_prof_mu);
+    g_prof_pairs.emplace_back(a, b);
+    g_prof_work += work;
+}
 
 void set_error(const std::string &msg) { g_err = msg; }
 psml_status fail(psml_status st, const std::string &msg) {
@@ -64,6 +90,30 @@ using namespace psml;
 int32_t psml_abi_version(void) { return PSML_ABI_VERSION; }
 const char *psml_last_error(void) { return g_err.c_str(); }
 uint64_t psml_kernel_launch_count(void) { return g_launches.load(); }
+
+psml_status psml_prof_enable(int32_t cls) {
+    if (cls < -1 || cls > 5) return fail(PSML_ERR_INVALID, "profile class must be in [-1, 5]");
+    g_prof_cls.store(cls);
+    return PSML_OK;
+}
+
+psml_status psml_prof_read(double *total_ms, int64_t *launches, double *work) {
+    PSML_CUDA_TRY(cudaDeviceSynchronize());
+    std::lock_guard<std::mutex> lk(g_prof_mu);
+    double ms = 0;
+    for (auto &pr : g_prof_pairs) {
+        float t = 0;
+        if (cudaEventElapsedTime(&t, pr.first, pr.second) == cudaSuccess) ms += t;
+        g_prof_pool.push_back(pr.first);
+        g_prof_pool.push_back(pr.second);
+    }
+    if (total_ms) *total_ms = ms;
+    if (launches) *launches = (int64_t)g_prof_pairs.size();
+    if (work) *work = g_prof_work;
+    g_prof_pairs.clear();
+    g_prof_work = 0;
+    return PSML_OK;
+}
 
 psml_status psml_device_info(int32_t *sm_count, int32_t *cc_major, int32_t *cc_minor) {
     int dev = 0, n = 0;
@@ -189,36 +239,28 @@ psml_status psml_reconstruct(psml_ring ring, const void *x0, const void *x1, int
 template <typename T>
 static psml_status triplet_gen_t(Ctx *c, uint64_t seed, uint64_t cid, int64_t M, int64_t K, int64_t N,
                                  void *const U[2], void *const V[2], void *const Z[2], cudaStream_t s) {
-    // workspace: U sum (MK) + V sum (KN) + split-K partial (MN)
-    const int64_t words = M * K + K * N + M * N;
-    PSML_TRY(c->ensure_ws(sizeof(T) * words));
-    T *Us = (T *)c->ws, *Vs = Us + M * K, *part = Vs + K * N;
     dealer_pair_kernel<T><<<grid_for(M * K / 8 + 1, 256), 256, 0, s>>>(make_key(seed, TAG_U0, cid), make_key(seed, TAG_U1, cid), M * K,
-                                                                       (T *)U[0], (T *)U[1], Us);
+                                                                       (T *)U[0], (T *)U[1], nullptr);
     PSML_LAUNCH_CHECK();
     dealer_pair_kernel<T><<<grid_for(K * N / 8 + 1, 256), 256, 0, s>>>(make_key(seed, TAG_V0, cid), make_key(seed, TAG_V1, cid), K * N,
-                                                                       (T *)V[0], (T *)V[1], Vs);
+                                                                       (T *)V[0], (T *)V[1], nullptr);
     PSML_LAUNCH_CHECK();
-    // Z = (U0+U1)(V0+V1): through the plain ring GEMM (tcgen05 when it pays), then the split
+    prg_kernel<T, 0><<<grid_for(M * N / 8 + 2, 256), 256, 0, s>>>(make_key(seed, TAG_Z0, cid), 0, M * N, (T *)Z[0],
+                                                                  nullptr, nullptr);
+    PSML_LAUNCH_CHECK();
+    // Z = (U0+U1)(V0+V1) on the tensor cores where it pays, else the CUDA-core ring GEMM
     if (c->use_tc(M, K, N)) {
-        size_t need = tc_ring_gemm_ws_bytes(8 * (int)sizeof(T), M, K, N);
-        // plain GEMM into Z[1], then Z0 = PRG, Z1 -= Z0 (fused tiny kernel)
-        PSML_TRY(c->ensure_ws(sizeof(T) * words + need));
-        Us = (T *)c->ws; Vs = Us + M * K;
-        psml_status st = tc_ring_gemm_plain(8 * (int)sizeof(T), Us, Vs, M, K, N, Z[1],
-                                            (char *)c->ws + sizeof(T) * words, need, s);
-        if (st == PSML_OK) {
-            prg_kernel<T, 1><<<grid_for(M * N / 8 + 2, 256), 256, 0, s>>>(make_key(seed, TAG_Z0, cid), 0, M * N, (T *)Z[0],
-                                                                          (const T *)Z[1], (T *)Z[1]);
-            PSML_LAUNCH_CHECK();
-            return PSML_OK;
-        }
+        const size_t need = tc_ring_gemm_ws_bytes(8 * (int)sizeof(T), M, K, N);
+        PSML_TRY(c->ensure_ws(need));
+        psml_status st = tc_dealer_gemm(8 * (int)sizeof(T), U[0], U[1], V[0], V[1], M, K, N, Z[0], Z[1], c->ws,
+                                        c->ws_bytes, s);
         if (st != PSML_ERR_UNSUPPORTED) return st;
     }
+    PSML_TRY(c->ensure_ws(sizeof(T) * M * N));
+    T *part = (T *)c->ws;
     DealerOps<T> ops;
     ops.U0 = (const T *)U[0]; ops.U1 = (const T *)U[1]; ops.V0 = (const T *)V[0]; ops.V1 = (const T *)V[1];
-    ops.Z0 = (T *)Z[0]; ops.Z1 = (T *)Z[1];
-    ops.kz0 = make_key(seed, TAG_Z0, cid);
+    ops.Z0 = (const T *)Z[0]; ops.Z1 = (T *)Z[1];
     ops.M = M; ops.N = N; ops.Kext = K;
     return launch_ring_gemm<T, DealerOps<T>>(ops, part, M * N, s, c->sm_count);
 }

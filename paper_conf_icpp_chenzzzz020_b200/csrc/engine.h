@@ -67,6 +67,9 @@ psml_status trace_opened(Ctx *c, int64_t M, int64_t K, int64_t N, const psml_tra
     return PSML_OK;
 }
 
+psml_status tc_dealer_gemm(int l, const void *U0, const void *U1, const void *V0, const void *V1, int64_t M, int64_t K,
+                           int64_t N, const void *Z0, void *Z1, void *ws, size_t ws_bytes, cudaStream_t s);
+
 // tcgen05 Beaver product (gemm_tc.cu); PSML_ERR_UNSUPPORTED = take the CUDA-core path.
 template <typename T>
 psml_status tc_beaver_matmul(Ctx *c, const T *const A[2], const T *const B[2], const T *const U[2],

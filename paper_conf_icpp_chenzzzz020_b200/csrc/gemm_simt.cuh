@@ -32,12 +32,13 @@ struct PlainOps {
     __device__ __forceinline__ void store(int, int64_t m, int64_t n, T acc) const { C[m * N + n] = acc; }
 };
 
-// Dealer: Z = (U_0 + U_1)(V_0 + V_1); Z_0 = PRG("Z0"), Z_1 = Z - Z_0 (Eqs. 2-3, R4).
+// Dealer: Z = (U_0 + U_1)(V_0 + V_1); Z_1 = Z - Z_0 with Z_0 = PRG("Z0") already written by the
+// vectorised PRG kernel (Eqs. 2-3, R4).
 template <typename T>
 struct DealerOps {
     const T *U0, *U1, *V0, *V1;
-    T *Z0, *Z1;
-    PrgKey kz0;
+    const T *Z0;
+    T *Z1;
     int64_t M, N, Kext;
     static constexpr int nparty = 1;
     __device__ __forceinline__ T a(int, int64_t m, int64_t k) const {
@@ -47,9 +48,7 @@ struct DealerOps {
         return V0[k * N + n] + V1[k * N + n];
     }
     __device__ __forceinline__ void store(int, int64_t m, int64_t n, T acc) const {
-        T z0 = prg_elem<T>(kz0, (uint64_t)(m * N + n));
-        Z0[m * N + n] = z0;
-        Z1[m * N + n] = acc - z0;
+        Z1[m * N + n] = acc - Z0[m * N + n];
     }
 };
 
@@ -140,8 +139,8 @@ struct ConvBeaverOps {
 template <typename T>
 struct ConvDealerOps {
     const T *U0, *U1, *V0, *V1;
-    T *Z0, *Z1;
-    PrgKey kz0;
+    const T *Z0;
+    T *Z1;
     ConvGeom g;
     int64_t M, N, Kext;
     int transposed;
@@ -163,9 +162,7 @@ struct ConvDealerOps {
         return V0[k * N + n] + V1[k * N + n];
     }
     __device__ __forceinline__ void store(int, int64_t m, int64_t n, T acc) const {
-        T z0 = prg_elem<T>(kz0, (uint64_t)(m * N + n));
-        Z0[m * N + n] = z0;
-        Z1[m * N + n] = acc - z0;
+        Z1[m * N + n] = acc - Z0[m * N + n];
     }
 };
 
@@ -348,21 +345,18 @@ psml_status launch_ring_gemm(const Ops &ops, T *ws, int64_t ws_words, cudaStream
     const int64_t M = ops.M, N = ops.N, Kx = ops.Kext;
     if (M <= 0 || N <= 0) return PSML_OK;
     const int64_t outs = M * N * Ops::nparty;
+    // split-K so the grid fills the GPU: ~2 CTAs (tiled) or ~16 warps (GEMV) per SM, each split
+    // still >= 64 (tiled) / 256 (GEMV) deep.  Ring addition is exact, so partials are summed
+    // with uint64/uint32 atomics and the epilogue runs once in ring_gemm_finalize.
     int splits = 1;
     if (N <= 16) {
         const int64_t warps = M * Ops::nparty;
-        const int64_t target = (int64_t)sm_count * 32;
-        if (warps < target && Kx >= 2048) {
-            splits = (int)std::min<int64_t>((target + warps - 1) / warps, Kx / 512);
-            if (splits < 1) splits = 1;
-        }
+        const int64_t target = (int64_t)sm_count * 16;
+        if (warps < target) splits = (int)std::max<int64_t>(1, std::min<int64_t>((target + warps - 1) / warps, Kx / 256));
     } else {
         const int64_t tiles = ((M + 63) / 64) * ((N + 63) / 64) * Ops::nparty;
         const int64_t target = (int64_t)sm_count * 2;
-        if (tiles < target && Kx >= 1024) {
-            splits = (int)std::min<int64_t>((target + tiles - 1) / tiles, Kx / 256);
-            if (splits < 1) splits = 1;
-        }
+        if (tiles < target) splits = (int)std::max<int64_t>(1, std::min<int64_t>((target + tiles - 1) / tiles, Kx / 64));
     }
     if (splits > 1 && (ws == nullptr || ws_words < outs)) splits = 1;  // no workspace: no split
     T *partial = nullptr;
@@ -371,6 +365,7 @@ psml_status launch_ring_gemm(const Ops &ops, T *ws, int64_t ws_words, cudaStream
         PSML_CUDA_TRY(cudaMemsetAsync(partial, 0, sizeof(T) * outs, stream));
     }
     int64_t kps = (Kx + splits - 1) / splits;
+    ProfScope prof(PROF_GEMM, stream, (double)M * N * Kx * Ops::nparty);
     if (N <= 16) {
         const int64_t warps = M * Ops::nparty * splits;
         const int blocks = (int)((warps * 32 + 255) / 256);

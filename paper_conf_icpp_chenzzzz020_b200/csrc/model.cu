@@ -218,6 +218,7 @@ static int64_t ws_need(psml_model_s *m) {
 // ------------------------------------------------------------------------------------------------
 static psml_status deal_item(psml_model_s *m, DealItem &it, uint32_t step, cudaStream_t s) {
     const uint64_t seed = m->d.dealer_seed;
+    ProfScope prof(PROF_DEALER, s, (double)sizeof(T) * 2 * (it.U.n + it.V.n + it.Z.n + it.mat.n));
     const uint64_t cid = call_id(m->d.pair_id, step, it.layer, it.op, it.slot);
     switch (it.kind) {
     case IT_MATRIX: {
@@ -227,9 +228,12 @@ static psml_status deal_item(psml_model_s *m, DealItem &it, uint32_t step, cudaS
         dealer_pair_kernel<T><<<grid_for(it.K * it.N / 8 + 1, 256), 256, 0, s>>>(
             make_key(seed, TAG_V0, cid), make_key(seed, TAG_V1, cid), it.K * it.N, it.V.p[0], it.V.p[1], nullptr);
         PSML_LAUNCH_CHECK();
+        prg_kernel<T, 0><<<grid_for(it.M * it.N / 8 + 2, 256), 256, 0, s>>>(make_key(seed, TAG_Z0, cid), 0,
+                                                                            it.M * it.N, it.Z.p[0], nullptr, nullptr);
+        PSML_LAUNCH_CHECK();
         DealerOps<T> ops;
         ops.U0 = it.U.p[0]; ops.U1 = it.U.p[1]; ops.V0 = it.V.p[0]; ops.V1 = it.V.p[1];
-        ops.Z0 = it.Z.p[0]; ops.Z1 = it.Z.p[1]; ops.kz0 = make_key(seed, TAG_Z0, cid);
+        ops.Z0 = it.Z.p[0]; ops.Z1 = it.Z.p[1];
         ops.M = it.M; ops.N = it.N; ops.Kext = it.K;
         return launch_ring_gemm<T, DealerOps<T>>(ops, m->ws, m->ws_words, s, m->ctx->sm_count);
     }
@@ -242,9 +246,12 @@ static psml_status deal_item(psml_model_s *m, DealItem &it, uint32_t step, cudaS
         dealer_pair_kernel<T><<<grid_for(it.K * it.N / 8 + 1, 256), 256, 0, s>>>(
             make_key(seed, TAG_V0, cid), make_key(seed, TAG_V1, cid), it.K * it.N, it.V.p[0], it.V.p[1], nullptr);
         PSML_LAUNCH_CHECK();
+        prg_kernel<T, 0><<<grid_for(it.M * it.N / 8 + 2, 256), 256, 0, s>>>(make_key(seed, TAG_Z0, cid), 0,
+                                                                            it.M * it.N, it.Z.p[0], nullptr, nullptr);
+        PSML_LAUNCH_CHECK();
         ConvDealerOps<T> ops;
         ops.U0 = it.U.p[0]; ops.U1 = it.U.p[1]; ops.V0 = it.V.p[0]; ops.V1 = it.V.p[1];
-        ops.Z0 = it.Z.p[0]; ops.Z1 = it.Z.p[1]; ops.kz0 = make_key(seed, TAG_Z0, cid);
+        ops.Z0 = it.Z.p[0]; ops.Z1 = it.Z.p[1];
         ops.g = m->g; ops.M = it.M; ops.N = it.N; ops.Kext = it.K; ops.transposed = it.kind == IT_CONV_GW;
         return launch_ring_gemm<T, ConvDealerOps<T>>(ops, m->ws, m->ws_words, s, m->ctx->sm_count);
     }
@@ -521,6 +528,14 @@ psml_status psml_train_forward_backward(psml_model m, const void *const X[2], co
     PSML_TRY(forward(m, (const T *const *)X, (const T *const *)Y, nullptr, s));
     PSML_TRY(backward(m, s));
     m->grads_ready = true;
+    return PSML_OK;
+}
+
+psml_status psml_model_output(psml_model m, void **yhat0, void **yhat1, int64_t *n) {
+    if (!m) return fail(PSML_ERR_INVALID, "model is null");
+    if (yhat0) *yhat0 = m->yhat.p[0];
+    if (yhat1) *yhat1 = m->yhat.p[1];
+    if (n) *n = m->yhat.n;
     return PSML_OK;
 }
 

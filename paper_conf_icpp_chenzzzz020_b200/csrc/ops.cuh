@@ -47,8 +47,11 @@ psml_status beaver_matmul(const T *const A[2], const T *const B[2], const T *con
     jobs.j[3] = {B[1], V[1], mF1, K, N, tB};
     jobs.count = 4;
     const int64_t maxt = std::max(((M + 31) / 32) * ((K + 31) / 32), ((K + 31) / 32) * ((N + 31) / 32));
-    mask_kernel<T><<<dim3((unsigned)std::min<int64_t>(maxt, 148 * 8), 1, 4), dim3(32, 8), 0, s>>>(jobs);
-    PSML_LAUNCH_CHECK();
+    {
+        ProfScope prof(PROF_MASK, s, 3.0 * sizeof(T) * 2 * (M * K + K * N));
+        mask_kernel<T><<<dim3((unsigned)std::min<int64_t>(maxt, 148 * 8), 1, 4), dim3(32, 8), 0, s>>>(jobs);
+        PSML_LAUNCH_CHECK();
+    }
     BeaverOps<T> ops;
     ops.mE0 = mE0; ops.mE1 = mE1; ops.mF0 = mF0; ops.mF1 = mF1;
     for (int p = 0; p < 2; ++p) {
@@ -116,6 +119,9 @@ psml_status beaver_hadamard(const T *const A[2], const T *const B[2], const T *c
                             const T *const V[2], const T *const Z[2], int64_t n, int trunc,
                             T *const C[2], T *ws, cudaStream_t s) {
     Pair<T> mE{{ws, ws + n}}, mF{{ws + 2 * n, ws + 3 * n}};
+    // algorithmic bytes: round 1 reads A,B,U,V writes E,F (6 words/party); round 2 reads
+    // E_0,E_1,F_0,F_1,U,V,Z writes C (4 + 4 per party)
+    ProfScope prof(PROF_HAD, s, (double)sizeof(T) * n * (12 + 12));
     CPair<T> a{{A[0], A[1]}}, b{{B[0], B[1]}}, u{{U[0], U[1]}}, v{{V[0], V[1]}}, z{{Z[0], Z[1]}};
     hadamard_mask_kernel<T><<<ew_grid(n), EW_THREADS, 0, s>>>(a, b, u, v, n, mE, mF);
     PSML_LAUNCH_CHECK();
@@ -147,6 +153,9 @@ psml_status msb_chain(const T *const x[2], int64_t n, const T *const mat[2], int
     a.msg = Pair<T>{{ws + 4 * n, ws + 8 * n}};
     a.n = n; a.mode = mode; a.half = half; a.L = ilog2_int(l); a.l = l;
     const int g = ew_grid(n);
+    // algorithmic bytes of the chain (both parties): per AND round each party reads 2 message
+    // words of both parties + 3 material words + state and writes state + 2 messages
+    ProfScope prof(PROF_MSB, s, (double)sizeof(T) * n * (2.0 * (a.L + 2) * 14 + 16));
     msb_round0_kernel<T><<<g, EW_THREADS, 0, s>>>(a);
     PSML_LAUNCH_CHECK();
     for (int j = 1; j <= a.L; ++j) {

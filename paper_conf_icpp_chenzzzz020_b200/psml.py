@@ -51,6 +51,8 @@ _SIGS = {
     "psml_last_error": (ctypes.c_char_p, []),
     "psml_device_info": (i32, [vp, vp, vp]),
     "psml_kernel_launch_count": (u64, []),
+    "psml_prof_enable": (i32, [i32]),
+    "psml_prof_read": (i32, [vp, vp, vp]),
     "psml_ctx_create": (i32, [Ring, i32, vp]),
     "psml_ctx_destroy": (i32, [vp]),
     "psml_prg_fill": (i32, [Ring, u64, u32, u64, u64, i64, vp, vp]),
@@ -79,6 +81,7 @@ _SIGS = {
     "psml_model_deal": (i32, [vp, u32, i32, vp]),
     "psml_secure_train_step": (i32, [vp, P2, P2, u32, vp]),
     "psml_train_forward_backward": (i32, [vp, P2, P2, u32, vp]),
+    "psml_model_output": (i32, [vp, vp, vp, vp]),
     "psml_model_grads": (i32, [vp, vp, vp]),
     "psml_train_apply_update": (i32, [vp, i32, vp]),
     "psml_secure_infer": (i32, [vp, P2, u32, P2, vp]),
@@ -162,6 +165,21 @@ def abi_version():
 
 def kernel_launch_count():
     return lib().psml_kernel_launch_count()
+
+
+PROF_GEMM, PROF_TC, PROF_MSB, PROF_HAD, PROF_DEALER, PROF_MASK = range(6)
+
+
+def prof_enable(cls):
+    """Time every library launch of kernel class `cls` with CUDA events (-1 disables)."""
+    _call("psml_prof_enable", cls)
+
+
+def prof_read():
+    """(total ms, launches, algorithmic work) of the profiled class since the last read."""
+    ms, n, w = ctypes.c_double(), i64(), ctypes.c_double()
+    _call("psml_prof_read", ctypes.byref(ms), ctypes.byref(n), ctypes.byref(w))
+    return ms.value, n.value, w.value
 
 
 def device_info():
@@ -389,6 +407,12 @@ class Model:
     def forward_backward(self, X, Y, step, stream=None):
         _call("psml_train_forward_backward", self.handle, _pair(X), _pair(Y), step,
               _stream(stream))
+
+    def output(self):
+        """Model-owned prediction shares (ptr0, ptr1, words) of the last forward pass."""
+        a, b, n = vp(), vp(), i64()
+        _call("psml_model_output", self.handle, ctypes.byref(a), ctypes.byref(b), ctypes.byref(n))
+        return a.value, b.value, n.value
 
     def grads(self):
         """(pointer, words per party) of the model-owned [2][P] gradient buffer."""

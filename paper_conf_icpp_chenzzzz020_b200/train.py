@@ -89,6 +89,11 @@ class SecureTrainer:
             raise ValueError("data-parallel pair count must be a power of two (R16)")
         self.model.apply_update(extra_shift=extra)
 
+    def last_yhat(self):
+        """Prediction shares of the last step as two uint64 views of model-owned memory."""
+        a, b, n = self.model.output()
+        return _wrap_device_ptr(a, n, "<u8"), _wrap_device_ptr(b, n, "<u8")
+
     def grad_tensor(self):
         """int64 view of the model-owned [2][P] gradient buffer (for the all-reduce)."""
         ptr, words = self.model.grads()
@@ -114,9 +119,9 @@ class SecureTrainer:
         self.ctx.close()
 
 
-def _wrap_device_ptr(ptr, numel):
-    """A torch int64 tensor aliasing `numel` words of library-owned device memory."""
+def _wrap_device_ptr(ptr, numel, typestr="<i8"):
+    """A torch tensor aliasing `numel` 8-byte words of library-owned device memory."""
     class _Holder:
-        __cuda_array_interface__ = {"shape": (numel,), "typestr": "<i8", "data": (ptr, False),
+        __cuda_array_interface__ = {"shape": (numel,), "typestr": typestr, "data": (ptr, False),
                                     "version": 3, "strides": None}
     return torch.as_tensor(_Holder(), device="cuda")
