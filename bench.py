@@ -154,6 +154,14 @@ def bench_ours(args):
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream()
 
+    def graph_step(s, X, Y):
+        # client encode + share into the captured buffers, then one graph replay (dealer +
+        # online step [+ update]); data parallel: NCCL all-reduce of gradient shares + update
+        tr.graph_step(X, Y, s)
+        if world > 1:
+            dist.all_reduce(tr.grad_tensor(), op=dist.ReduceOp.SUM)
+            tr.model.apply_update(extra_shift=int(round(np.log2(world))))
+
     def one_step(s, X, Y, online_only=False, shares=None):
         if online_only:
             tr.model.train_step(*shares, s) if world == 1 else tr.step_dp(*shares, s, deal=False)
@@ -183,9 +191,16 @@ def bench_ours(args):
     for s in range(W):
         one_step(s, Xs[s], Ys[s])
     torch.cuda.synchronize()
+    EB = 10 ** 6   # eager comparison steps use their own step ids (fresh dealer material)
+    t_eager = max_over_ranks(timed(lambda s: one_step(s, Xs[(s - EB) % nb], Ys[(s - EB) % nb]), K, EB),
+                             world)
+    tr.capture(with_update=(world == 1))
+    graph_step(W, Xs[0], Ys[0])        # warm the graph once
+    torch.cuda.synchronize()
     l0 = psml.kernel_launch_count()
+    n_nodes = tr.graph_kernel_nodes()
     with ClockSampler(local) as clk:
-        t_dev = timed(lambda s: one_step(s, Xs[s], Ys[s]), K, W)
+        t_dev = timed(lambda s: graph_step(s, Xs[s], Ys[s]), K, W)
     launches = psml.kernel_launch_count() - l0
     t_dev = max_over_ranks(t_dev, world)
 
@@ -213,7 +228,7 @@ def bench_ours(args):
         i = (s - 2 * (W + K)) % nb
         X = Xh[i].to(dev, non_blocking=True)
         Y = Yh[i].to(dev, non_blocking=True)
-        one_step(s, X, Y)
+        graph_step(s, X, Y)
         # the step's result: both parties' prediction shares of this batch
         y0, y1 = tr.last_yhat()
         out_host[0].view(-1).copy_(y0, non_blocking=True)
@@ -231,6 +246,10 @@ def bench_ours(args):
                    "l2": "256 MiB flush between timed steps (outside the events)",
                    "step": "client encode+share, dealer (offline), online secure step"},
         "online_samples_per_s": samples / t_on,
+        "eager_samples_per_s": samples / t_eager,
+        "cuda_graph": {"kernel_nodes_per_step": n_nodes,
+                       "note": "value/e2e replay one captured graph per step (dealer + online "
+                               "step + update); online/eager figures use per-kernel launches"},
         "e2e": {"value": samples / t_e2e, "unit": "samples/s", "h2d_bytes_per_step": h2d,
                 "d2h_bytes_per_step": d2h},
         "gpu_launches": int(launches),

@@ -258,6 +258,17 @@ psml_status psml_model_grads(psml_model model, void **grads, int64_t *words_per_
 /* W^m_i -= trunc_i(gradW_i, 26 + lr_shift - m + extra_shift); W_i = trunc_i(W^m_i, m - f).
  * extra_shift = log2(number of data-parallel pairs summed into the gradient). */
 psml_status psml_train_apply_update(psml_model model, int32_t extra_shift, psml_stream stream);
+/* CUDA-graph fast path.  Capture ONE training step on `stream` (must not be the legacy default
+ * stream) reading the minibatch shares from the fixed device buffers X[2], Y[2]: flags bit 0 =
+ * include the dealer (offline material), bit 1 = include the update.  The dealer's call ids take
+ * their step field from a model-owned device word, so the same graph serves every step.
+ * psml_model_step_graph writes step_id to that word and launches the graph; the caller refills
+ * X/Y before each replay.  Capture must not overlap other work on the stream. */
+psml_status psml_model_capture_step(psml_model model, const void *const X[2], const void *const Y[2],
+                                    int32_t flags, psml_stream stream);
+psml_status psml_model_step_graph(psml_model model, uint32_t step_id, psml_stream stream);
+/* Number of kernel nodes in the captured step graph (launch accounting for bench.py). */
+psml_status psml_model_graph_nodes(psml_model model, int64_t *n);
 /* Secure inference (the forward half): Yhat[i]: batch x d_L.  Needs
  * psml_model_deal(step_id, infer_only=1) (or a full deal) for the same step_id. */
 psml_status psml_secure_infer(psml_model model, const void *const X[2], uint32_t step_id,

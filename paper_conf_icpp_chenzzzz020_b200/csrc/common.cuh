@@ -95,12 +95,26 @@ __device__ __forceinline__ uint32_t rotl(uint32_t v, int c) { return __funnelshi
 struct PrgKey {
     uint32_t k0, k1;         // seed words (rest of the 256-bit key is zero)
     uint32_t n0, n1, n2;     // nonce = tag || call_id
+    const uint32_t *step;    // optional: device word overriding call-id bits 55:24 (CUDA graphs)
 };
 
-__host__ __device__ inline PrgKey make_key(uint64_t seed, uint32_t tag, uint64_t call_id) {
+__host__ __device__ inline PrgKey make_key(uint64_t seed, uint32_t tag, uint64_t call_id,
+                                           const uint32_t *step = nullptr) {
     PrgKey k;
     k.k0 = (uint32_t)seed; k.k1 = (uint32_t)(seed >> 32);
     k.n0 = tag; k.n1 = (uint32_t)call_id; k.n2 = (uint32_t)(call_id >> 32);
+    k.step = step;
+    return k;
+}
+
+// Resolve the step field from device memory (call id = pair|step|layer|op|slot, R11),
+// so a captured graph replays with a new step number without re-instantiation.
+__device__ __forceinline__ PrgKey live_key(PrgKey k) {
+    if (k.step) {
+        const uint32_t st = *k.step;
+        k.n1 = (k.n1 & 0x00FFFFFFu) | (st << 24);
+        k.n2 = (k.n2 & 0xFF000000u) | (st >> 8);
+    }
     return k;
 }
 

@@ -32,22 +32,23 @@ struct Ctx {
 // ------------------------------------------------------------------------------------------------
 template <typename T>
 psml_status hadamard_triplet_launch(uint64_t seed, uint64_t cid, int64_t n, void *const U[2], void *const V[2],
-                                    void *const Z[2], cudaStream_t s) {
+                                    void *const Z[2], cudaStream_t s, const uint32_t *step = nullptr) {
     Pair<T> u{{(T *)U[0], (T *)U[1]}}, v{{(T *)V[0], (T *)V[1]}}, z{{(T *)Z[0], (T *)Z[1]}};
     const int64_t nblk = (n + PerBlock<T>::value - 1) / PerBlock<T>::value;
     hadamard_triplet_kernel<T><<<grid_for(nblk, 128, 148 * 32), 128, 0, s>>>(
-        make_key(seed, TAG_U0, cid), make_key(seed, TAG_U1, cid), make_key(seed, TAG_V0, cid),
-        make_key(seed, TAG_V1, cid), make_key(seed, TAG_Z0, cid), n, u, v, z);
+        make_key(seed, TAG_U0, cid, step), make_key(seed, TAG_U1, cid, step), make_key(seed, TAG_V0, cid, step),
+        make_key(seed, TAG_V1, cid, step), make_key(seed, TAG_Z0, cid, step), n, u, v, z);
     PSML_LAUNCH_CHECK();
     return PSML_OK;
 }
 
 template <typename T>
-psml_status msb_dealer_launch(uint64_t seed, uint64_t cid, int64_t n, void *const mat[2], cudaStream_t s) {
+psml_status msb_dealer_launch(uint64_t seed, uint64_t cid, int64_t n, void *const mat[2], cudaStream_t s,
+                              const uint32_t *step = nullptr) {
     const int L = ilog2_int(8 * (int)sizeof(T));
     const int64_t nblk = (n + PerBlock<T>::value - 1) / PerBlock<T>::value;
     dim3 grid((unsigned)grid_for(nblk, 128, 148 * 8), (unsigned)(2 * L + 1));
-    msb_dealer_kernel<T><<<grid, 128, 0, s>>>(seed, cid, n, L, (T *)mat[0], (T *)mat[1]);
+    msb_dealer_kernel<T><<<grid, 128, 0, s>>>(seed, cid, n, L, (T *)mat[0], (T *)mat[1], step);
     PSML_LAUNCH_CHECK();
     return PSML_OK;
 }

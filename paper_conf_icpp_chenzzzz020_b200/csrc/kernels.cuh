@@ -21,6 +21,7 @@ template <typename T, int OP>
 __global__ void prg_kernel(PrgKey key, uint64_t offset, int64_t n, T *__restrict__ out,
                            const T *__restrict__ x, T *__restrict__ out2) {
     constexpr int PB = PerBlock<T>::value;
+    key = live_key(key);
     const uint64_t first_blk = offset / PB;
     const uint64_t last_blk = (offset + (uint64_t)n - 1) / PB;
     for (uint64_t b = first_blk + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; b <= last_blk;
@@ -75,6 +76,8 @@ template <typename T>
 __global__ void dealer_pair_kernel(PrgKey k0, PrgKey k1, int64_t n, T *__restrict__ o0,
                                    T *__restrict__ o1, T *__restrict__ sum) {
     constexpr int PB = PerBlock<T>::value;
+    k0 = live_key(k0);
+    k1 = live_key(k1);
     const int64_t nblk = (n + PB - 1) / PB;
     for (int64_t b = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; b < nblk; b += (int64_t)gridDim.x * blockDim.x) {
         uint32_t w0[16], w1[16];
@@ -102,6 +105,7 @@ template <typename T>
 __global__ void hadamard_triplet_kernel(PrgKey ku0, PrgKey ku1, PrgKey kv0, PrgKey kv1, PrgKey kz0,
                                         int64_t n, Pair<T> U, Pair<T> V, Pair<T> Z) {
     constexpr int PB = PerBlock<T>::value;
+    ku0 = live_key(ku0); ku1 = live_key(ku1); kv0 = live_key(kv0); kv1 = live_key(kv1); kz0 = live_key(kz0);
     const int64_t nblk = (n + PB - 1) / PB;
     for (int64_t b = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; b < nblk; b += (int64_t)gridDim.x * blockDim.x) {
         uint32_t a0[16], a1[16], c0[16], c1[16], z[16];
@@ -125,8 +129,12 @@ __global__ void hadamard_triplet_kernel(PrgKey ku0, PrgKey ku1, PrgKey kv0, PrgK
 // MSB material: blockIdx.y = AND index t (0 .. 2L-1) or 2L for the daBit.
 template <typename T>
 __global__ void msb_dealer_kernel(uint64_t seed, uint64_t call_id, int64_t n, int L, T *__restrict__ m0,
-                                  T *__restrict__ m1) {
+                                  T *__restrict__ m1, const uint32_t *step) {
     constexpr int PB = PerBlock<T>::value;
+    if (step) {
+        const uint64_t st = *step;
+        call_id = (call_id & ~(0xFFFFFFFFull << 24)) | (st << 24);
+    }
     const int t = blockIdx.y;
     const int64_t nblk = (n + PB - 1) / PB;
     for (int64_t b = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; b < nblk; b += (int64_t)gridDim.x * blockDim.x) {

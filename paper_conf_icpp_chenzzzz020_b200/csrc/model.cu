@@ -25,6 +25,8 @@ using T = uint64_t;
 enum { OP_FWD = 0, OP_GRADW = 1, OP_GRADIN = 2, OP_RELU_MSB = 3, OP_EQ9_MSB = 4, OP_HADAMARD = 6 };
 enum ItemKind { IT_MATRIX, IT_CONV_FWD, IT_CONV_GW, IT_HAD, IT_MSB };
 
+__global__ void set_word_kernel(uint32_t *p, uint32_t v) { *p = v; }
+
 static inline uint64_t call_id(uint32_t pair, uint32_t step, int layer, int op, int slot) {
     return ((uint64_t)(pair & 0xFF) << 56) | ((uint64_t)step << 24) | ((uint64_t)(layer & 0xFF) << 16) |
            ((uint64_t)(op & 0xFF) << 8) | (uint64_t)(slot & 0xFF);
@@ -69,6 +71,10 @@ struct psml_model_s {
     int64_t dealt_step = -1;
     bool dealt_full = false;
     bool grads_ready = false;
+    uint32_t *step_dev = nullptr;      // device copy of the step number (dealer call ids)
+    cudaGraphExec_t graph = nullptr;   // captured step (psml_model_capture_step)
+    int graph_flags = 0;
+    int64_t graph_kernels = 0;
 };
 
 namespace psml {
@@ -223,12 +229,12 @@ static psml_status deal_item(psml_model_s *m, DealItem &it, uint32_t step, cudaS
     switch (it.kind) {
     case IT_MATRIX: {
         dealer_pair_kernel<T><<<grid_for(it.M * it.K / 8 + 1, 256), 256, 0, s>>>(
-            make_key(seed, TAG_U0, cid), make_key(seed, TAG_U1, cid), it.M * it.K, it.U.p[0], it.U.p[1], nullptr);
+            make_key(seed, TAG_U0, cid, m->step_dev), make_key(seed, TAG_U1, cid, m->step_dev), it.M * it.K, it.U.p[0], it.U.p[1], nullptr);
         PSML_LAUNCH_CHECK();
         dealer_pair_kernel<T><<<grid_for(it.K * it.N / 8 + 1, 256), 256, 0, s>>>(
-            make_key(seed, TAG_V0, cid), make_key(seed, TAG_V1, cid), it.K * it.N, it.V.p[0], it.V.p[1], nullptr);
+            make_key(seed, TAG_V0, cid, m->step_dev), make_key(seed, TAG_V1, cid, m->step_dev), it.K * it.N, it.V.p[0], it.V.p[1], nullptr);
         PSML_LAUNCH_CHECK();
-        prg_kernel<T, 0><<<grid_for(it.M * it.N / 8 + 2, 256), 256, 0, s>>>(make_key(seed, TAG_Z0, cid), 0,
+        prg_kernel<T, 0><<<grid_for(it.M * it.N / 8 + 2, 256), 256, 0, s>>>(make_key(seed, TAG_Z0, cid, m->step_dev), 0,
                                                                             it.M * it.N, it.Z.p[0], nullptr, nullptr);
         PSML_LAUNCH_CHECK();
         DealerOps<T> ops;
@@ -241,12 +247,12 @@ static psml_status deal_item(psml_model_s *m, DealItem &it, uint32_t step, cudaS
     case IT_CONV_GW: {
         const int64_t nin = it.U.n;
         dealer_pair_kernel<T><<<grid_for(nin / 8 + 1, 256), 256, 0, s>>>(
-            make_key(seed, TAG_U0, cid), make_key(seed, TAG_U1, cid), nin, it.U.p[0], it.U.p[1], nullptr);
+            make_key(seed, TAG_U0, cid, m->step_dev), make_key(seed, TAG_U1, cid, m->step_dev), nin, it.U.p[0], it.U.p[1], nullptr);
         PSML_LAUNCH_CHECK();
         dealer_pair_kernel<T><<<grid_for(it.K * it.N / 8 + 1, 256), 256, 0, s>>>(
-            make_key(seed, TAG_V0, cid), make_key(seed, TAG_V1, cid), it.K * it.N, it.V.p[0], it.V.p[1], nullptr);
+            make_key(seed, TAG_V0, cid, m->step_dev), make_key(seed, TAG_V1, cid, m->step_dev), it.K * it.N, it.V.p[0], it.V.p[1], nullptr);
         PSML_LAUNCH_CHECK();
-        prg_kernel<T, 0><<<grid_for(it.M * it.N / 8 + 2, 256), 256, 0, s>>>(make_key(seed, TAG_Z0, cid), 0,
+        prg_kernel<T, 0><<<grid_for(it.M * it.N / 8 + 2, 256), 256, 0, s>>>(make_key(seed, TAG_Z0, cid, m->step_dev), 0,
                                                                             it.M * it.N, it.Z.p[0], nullptr, nullptr);
         PSML_LAUNCH_CHECK();
         ConvDealerOps<T> ops;
@@ -257,11 +263,11 @@ static psml_status deal_item(psml_model_s *m, DealItem &it, uint32_t step, cudaS
     }
     case IT_HAD: {
         void *U[2] = {it.U.p[0], it.U.p[1]}, *V[2] = {it.V.p[0], it.V.p[1]}, *Z[2] = {it.Z.p[0], it.Z.p[1]};
-        return hadamard_triplet_launch<T>(seed, cid, it.n, U, V, Z, s);
+        return hadamard_triplet_launch<T>(seed, cid, it.n, U, V, Z, s, m->step_dev);
     }
     case IT_MSB: {
         void *mt[2] = {it.mat.p[0], it.mat.p[1]};
-        return msb_dealer_launch<T>(seed, cid, it.n, mt, s);
+        return msb_dealer_launch<T>(seed, cid, it.n, mt, s, m->step_dev);
     }
     }
     return PSML_OK;
@@ -462,6 +468,11 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
     PSML_TRY(balloc(mp, m->tmp, B * maxw));
     plan_items(mp);
     PSML_TRY(alloc_items(mp));
+    {
+        T *sd = nullptr;
+        PSML_TRY(dalloc(mp, &sd, 1));
+        m->step_dev = (uint32_t *)sd;
+    }
     m->ws_words = ws_need(mp);
     PSML_TRY(dalloc(mp, &m->ws, m->ws_words));
     *out = m.release();
@@ -471,6 +482,7 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
 psml_status psml_model_destroy(psml_model model) {
     if (!model) return PSML_OK;
     cudaDeviceSynchronize();
+    if (model->graph) cudaGraphExecDestroy(model->graph);
     for (void *p : model->allocs) cudaFree(p);
     delete model;
     return PSML_OK;
@@ -509,6 +521,8 @@ psml_status psml_model_get_master(psml_model m, int32_t layer, void *const Wm[2]
 psml_status psml_model_deal(psml_model m, uint32_t step_id, int32_t infer_only, psml_stream stream) {
     if (!m) return fail(PSML_ERR_INVALID, "model is null");
     cudaStream_t s = (cudaStream_t)stream;
+    set_word_kernel<<<1, 1, 0, s>>>(m->step_dev, step_id);
+    PSML_LAUNCH_CHECK();
     for (auto &it : m->items) {
         if (infer_only && !it.fwd) continue;
         PSML_TRY(deal_item(m, it, step_id, s));
@@ -571,6 +585,72 @@ psml_status psml_secure_train_step(psml_model m, const void *const X[2], const v
                                    psml_stream stream) {
     PSML_TRY(psml_train_forward_backward(m, X, Y, step_id, stream));
     return psml_train_apply_update(m, 0, stream);
+}
+
+psml_status psml_model_capture_step(psml_model m, const void *const X[2], const void *const Y[2], int32_t flags,
+                                   psml_stream stream) {
+    if (!m || !X || !Y) return fail(PSML_ERR_INVALID, "null argument");
+    PSML_TRY(check_ptrs({X[0], X[1], Y[0], Y[1]}));
+    if (flags & ~3) return fail(PSML_ERR_INVALID, "flags: bit 0 = with dealer, bit 1 = with update");
+    cudaStream_t s = (cudaStream_t)stream;
+    if (s == nullptr) return fail(PSML_ERR_INVALID, "capture needs a non-default stream");
+    if (m->graph) {
+        cudaGraphExecDestroy(m->graph);
+        m->graph = nullptr;
+    }
+    const int prof = g_prof_cls.exchange(-1);   // no profiling events inside the graph
+    PSML_CUDA_TRY(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
+    psml_status st = PSML_OK;
+    if (flags & 1)
+        for (auto &it : m->items)
+            if (st == PSML_OK) st = deal_item(m, it, 0, s);
+    if (st == PSML_OK) st = forward(m, (const T *const *)X, (const T *const *)Y, nullptr, s);
+    if (st == PSML_OK) st = backward(m, s);
+    if (st == PSML_OK && (flags & 2)) {
+        m->grads_ready = true;
+        st = psml_train_apply_update(m, 0, stream);
+    }
+    cudaGraph_t g = nullptr;
+    cudaError_t e = cudaStreamEndCapture(s, &g);
+    g_prof_cls.store(prof);
+    if (st != PSML_OK) {
+        if (g) cudaGraphDestroy(g);
+        return st;
+    }
+    if (e != cudaSuccess) return fail(PSML_ERR_CUDA, std::string("graph capture: ") + cudaGetErrorString(e));
+    size_t nn = 0;
+    cudaGraphGetNodes(g, nullptr, &nn);
+    std::vector<cudaGraphNode_t> nodes(nn);
+    if (nn) cudaGraphGetNodes(g, nodes.data(), &nn);
+    m->graph_kernels = 0;
+    for (auto nd : nodes) {
+        cudaGraphNodeType t;
+        if (cudaGraphNodeGetType(nd, &t) == cudaSuccess && t == cudaGraphNodeTypeKernel) ++m->graph_kernels;
+    }
+    e = cudaGraphInstantiate(&m->graph, g, 0);
+    cudaGraphDestroy(g);
+    if (e != cudaSuccess) return fail(PSML_ERR_CUDA, std::string("graph instantiate: ") + cudaGetErrorString(e));
+    m->graph_flags = flags;
+    return PSML_OK;
+}
+
+psml_status psml_model_graph_nodes(psml_model m, int64_t *n) {
+    if (!m || !n) return fail(PSML_ERR_INVALID, "null argument");
+    *n = m->graph_kernels + 1;   // + the step-word kernel launched before each replay
+    return PSML_OK;
+}
+
+psml_status psml_model_step_graph(psml_model m, uint32_t step_id, psml_stream stream) {
+    if (!m) return fail(PSML_ERR_INVALID, "model is null");
+    if (!m->graph) return fail(PSML_ERR_STATE, "no captured step: call psml_model_capture_step first");
+    cudaStream_t s = (cudaStream_t)stream;
+    set_word_kernel<<<1, 1, 0, s>>>(m->step_dev, step_id);
+    PSML_LAUNCH_CHECK();
+    PSML_CUDA_TRY(cudaGraphLaunch(m->graph, s));
+    g_launches.fetch_add((uint64_t)m->graph_kernels);   // the graph's kernels are our launches
+    if (m->graph_flags & 1) { m->dealt_step = step_id; m->dealt_full = true; }
+    m->grads_ready = !(m->graph_flags & 2);
+    return PSML_OK;
 }
 
 psml_status psml_secure_infer(psml_model m, const void *const X[2], uint32_t step_id, void *const Yhat[2],

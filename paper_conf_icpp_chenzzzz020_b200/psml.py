@@ -85,6 +85,9 @@ _SIGS = {
     "psml_model_grads": (i32, [vp, vp, vp]),
     "psml_train_apply_update": (i32, [vp, i32, vp]),
     "psml_secure_infer": (i32, [vp, P2, u32, P2, vp]),
+    "psml_model_capture_step": (i32, [vp, P2, P2, i32, vp]),
+    "psml_model_step_graph": (i32, [vp, u32, vp]),
+    "psml_model_graph_nodes": (i32, [vp, vp]),
 }
 EXPORTS = tuple(_SIGS)
 
@@ -422,6 +425,19 @@ class Model:
 
     def apply_update(self, extra_shift=0, stream=None):
         _call("psml_train_apply_update", self.handle, extra_shift, _stream(stream))
+
+    def capture_step(self, X, Y, with_deal=True, with_update=True, stream=None):
+        """Capture one step into a CUDA graph reading the fixed share buffers X, Y."""
+        flags = (1 if with_deal else 0) | (2 if with_update else 0)
+        _call("psml_model_capture_step", self.handle, _pair(X), _pair(Y), flags, _stream(stream))
+
+    def graph_nodes(self):
+        n = i64()
+        _call("psml_model_graph_nodes", self.handle, ctypes.byref(n))
+        return n.value
+
+    def step_graph(self, step, stream=None):
+        _call("psml_model_step_graph", self.handle, step, _stream(stream))
 
     def infer(self, X, step, out_shape, stream=None):
         Y = empty_pair(out_shape, self.ctx.l)

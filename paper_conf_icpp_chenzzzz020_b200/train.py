@@ -62,6 +62,33 @@ class SecureTrainer:
         return Xs, Ys
 
     # --- steps --------------------------------------------------------------------------------
+    def capture(self, with_update=True):
+        """Capture deal + online step (+ update) into a CUDA graph on a side stream; the batch is
+        shared into fixed buffers before each replay (graph_step)."""
+        d_in = self.model.layer_shape(0)[0] if self.task != "cnn" else 3 * 32 * 32
+        self.Xbuf = psml.empty_pair((self.batch, d_in), 64)
+        self.Ybuf = psml.empty_pair((self.batch, self.out_dim), 64)
+        for t in self.Xbuf + self.Ybuf:
+            t.zero_()
+        self.gstream = torch.cuda.Stream()
+        self.gstream.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.stream(self.gstream):
+            self.model.capture_step(self.Xbuf, self.Ybuf, with_deal=True, with_update=with_update,
+                                    stream=self.gstream)
+        torch.cuda.current_stream().wait_stream(self.gstream)
+        self.graph_update = with_update
+
+    def graph_kernel_nodes(self):
+        return self.model.graph_nodes()
+
+    def graph_step(self, X, Y, step):
+        """Client encode + share into the captured buffers, then replay the captured step."""
+        x = psml.encode(self.ring, torch.as_tensor(X, dtype=torch.float64))
+        y = psml.encode(self.ring, torch.as_tensor(Y, dtype=torch.float64))
+        psml.share(self.ring, SHARE_SEED, call_id(self.pair_id, step, 0, OP_SHARE, 0), x, out=self.Xbuf)
+        psml.share(self.ring, SHARE_SEED, call_id(self.pair_id, step, 0, OP_SHARE, 1), y, out=self.Ybuf)
+        self.model.step_graph(step)
+
     def deal(self, step, infer_only=False):
         self.model.deal(step, infer_only=infer_only)
 

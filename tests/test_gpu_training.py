@@ -77,3 +77,23 @@ def test_one_epoch_within_2pow_minus12_of_fp64(T, task, tol_log2):
     print(f"{task}: one-epoch max |w - w_fp64| = 2^{np.log2(err):.2f}")
     assert err < 2.0 ** tol_log2
     tr.close()
+
+
+@pytest.mark.parametrize("task,steps", [("mlp", 3), ("logreg", 2)])
+def test_graph_replay_bitexact_vs_oracle(T, task, steps):
+    """The captured CUDA graph (dealer + online step + update, step id from a device word)
+    reproduces the oracle's shares exactly for successive step ids."""
+    Wi = synth.init_weights(task)
+    tr = T.SecureTrainer(task, Wi, backend=0)
+    om = OP.Model(task, Wi)
+    X, Y = synth.batch(task, 0)
+    tr.step(torch.from_numpy(X), torch.from_numpy(Y), 0)      # eager warm-up step 0
+    OP.train_step(om, X, Y, 0)
+    tr.capture()
+    for s in range(1, steps + 1):
+        X, Y = synth.batch(task, s)
+        tr.graph_step(torch.from_numpy(X), torch.from_numpy(Y), s)
+        OP.train_step(om, X, Y, s)
+        torch.cuda.synchronize()
+        _compare_shares(tr, om)
+    tr.close()
