@@ -260,10 +260,14 @@ psml_status psml_model_grads(psml_model model, void **grads, int64_t *words_per_
 psml_status psml_train_apply_update(psml_model model, int32_t extra_shift, psml_stream stream);
 /* CUDA-graph fast path.  Capture ONE training step on `stream` (must not be the legacy default
  * stream) reading the minibatch shares from the fixed device buffers X[2], Y[2]: flags bit 0 =
- * include the dealer (offline material), bit 1 = include the update.  The dealer's call ids take
- * their step field from a model-owned device word, so the same graph serves every step.
- * psml_model_step_graph writes step_id to that word and launches the graph; the caller refills
- * X/Y before each replay.  Capture must not overlap other work on the stream. */
+ * include the dealer (offline material), bit 1 = include the update, bit 2 = PIPELINED dealer:
+ * the dealer pools are double-buffered (step s reads pool s % 2) and the graph of step s runs the
+ * dealer of step s + 1 on a forked stream concurrently with the online phase of step s (the first
+ * step's pool must be filled with psml_model_deal).  The dealer's call ids take their step field
+ * from a model-owned device word, so the same graph(s) serve every step.
+ * psml_model_step_graph writes the step word and launches the graph; the caller refills X/Y
+ * before each replay; pipelined steps must be consecutive (PSML_ERR_STATE otherwise).
+ * Capture must not overlap other work on the stream. */
 psml_status psml_model_capture_step(psml_model model, const void *const X[2], const void *const Y[2],
                                     int32_t flags, psml_stream stream);
 psml_status psml_model_step_graph(psml_model model, uint32_t step_id, psml_stream stream);

@@ -51,6 +51,9 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
         "r"(parity)
         : "memory");
 }
+__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
 __device__ __forceinline__ void bulk_g2s(uint32_t dst, const void *src, uint32_t bytes, uint32_t bar) {
     asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
                  "l"(src), "r"(bytes), "r"(bar)
@@ -312,6 +315,190 @@ __global__ void __launch_bounds__(128, 1) tc_ring_gemm_kernel(const TcParams<T> 
     if (warp == 2) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tmem));
 }
 
+// ------------------------------------------------------------------------------------------------
+// l = 64, v2: N = 128 per MMA, two shift-group passes over 4 TMEM accumulators of 128 columns.
+//   pass L: shifts 0..3 (10 limb pairs, limbs 0..3)   -> low  = sum_s S_s 2^{8s}        (exact)
+//   pass H: shifts 4..7 (26 limb pairs, limbs 0..7)   -> high = sum_s S_s 2^{8(s-4)} mod 2^32
+//   result = low + high * 2^32 mod 2^64.
+// Each MMA (128 x 128 x 32) reads 8 KB of smem per 64 tensor cycles instead of 6 KB per 32: the
+// v1 kernel was bound by the tensor core's shared-memory read path (ncu: tc smem wavefronts 80%).
+// Warps: 0 = TMA producer, 1 = MMA issuer, 2..5 = epilogue (warp w reads TMEM lanes 32 (w%4)..).
+// The pass-L result is staged in the output (or added to the split-K partial) and the pass-H
+// epilogue completes it; the pass-L drain overlaps the pass-H loads already in flight.
+// ------------------------------------------------------------------------------------------------
+template <int STAGES>
+__global__ void __launch_bounds__(192, 1) tc_ring_gemm64_v2(const TcParams<uint64_t> P) {
+    using T = uint64_t;
+    constexpr int BN = 128, L = 8;
+    extern __shared__ __align__(1024) uint8_t smem[];
+    constexpr int A_BYTES = BM * BK, B_BYTES = BN * BK;
+    constexpr int STAGE_BYTES = L * (A_BYTES + B_BYTES);
+    constexpr uint32_t IDESC = idesc_i8(BM, BN);
+    uint64_t *full = (uint64_t *)(smem + STAGES * STAGE_BYTES);
+    uint64_t *empty = full + STAGES;
+    uint64_t *accf = empty + STAGES;     // accumulators ready (phase 0: pass L, phase 1: pass H)
+    uint64_t *acce = accf + 1;           // pass-L accumulators drained
+    uint32_t *tmem_slot = (uint32_t *)(acce + 1);
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int party = blockIdx.z % P.nparty, split = blockIdx.z / P.nparty;
+    const int nb = blockIdx.x, rb = blockIdx.y;
+    const int nkb = P.nkb_lo + P.nkb_hi;
+    const int kb0 = split * P.kb_per_split;
+    const int kb1 = min(kb0 + P.kb_per_split, nkb);
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < STAGES; ++s) {
+            mbar_init(smem_u32(&full[s]), 1);
+            mbar_init(smem_u32(&empty[s]), 1);
+        }
+        mbar_init(smem_u32(accf), 1);
+        mbar_init(smem_u32(acce), 128);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if (warp == 2) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_u32(tmem_slot)));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem = *tmem_slot;
+
+    if (warp == 0) {
+        if (lane == 0) {
+            // ---------------- TMA producer: pass L (limbs 0..3), then pass H (limbs 0..7) ----------------
+            int stage = 0;
+            uint32_t phase = 0;
+            for (int pass = 0; pass < 2; ++pass) {
+                const int nl = pass == 0 ? 4 : 8;
+                for (int kb = kb0; kb < kb1; ++kb) {
+                    mbar_wait(smem_u32(&empty[stage]), phase ^ 1);
+                    const uint32_t fb = smem_u32(&full[stage]);
+                    mbar_expect_tx(fb, (uint32_t)(nl * (A_BYTES + B_BYTES)));
+                    const bool lo = kb < P.nkb_lo;
+                    const int kk = lo ? kb : kb - P.nkb_lo;
+                    const int nk = lo ? P.nkb_lo : P.nkb_hi;
+                    const uint8_t *a = (lo ? P.A_lo[party] : P.A_hi[party]) + ((int64_t)rb * nk + kk) * A_BYTES;
+                    const uint8_t *b = (lo ? P.B_lo[party] : P.B_hi[party]) + ((int64_t)nb * nk + kk) * B_BYTES;
+                    const int64_t as = lo ? P.a_stride_lo : P.a_stride_hi, bs = lo ? P.b_stride_lo : P.b_stride_hi;
+                    uint8_t *sa = smem + stage * STAGE_BYTES, *sb = sa + L * A_BYTES;
+                    for (int p = 0; p < nl; ++p) bulk_g2s(smem_u32(sa + p * A_BYTES), a + p * as, A_BYTES, fb);
+                    for (int q = 0; q < nl; ++q) bulk_g2s(smem_u32(sb + q * B_BYTES), b + q * bs, B_BYTES, fb);
+                    if (++stage == STAGES) { stage = 0; phase ^= 1; }
+                }
+            }
+        }
+    } else if (warp == 1) {
+        if (lane == 0) {
+            // ---------------- MMA issuer ----------------
+            int stage = 0;
+            uint32_t phase = 0;
+            for (int pass = 0; pass < 2; ++pass) {
+                if (pass == 1) {
+                    mbar_wait(smem_u32(acce), 0);   // epilogue has drained pass L
+                    tc_fence_after();
+                }
+                for (int kb = kb0; kb < kb1; ++kb) {
+                    mbar_wait(smem_u32(&full[stage]), phase);
+                    tc_fence_after();
+                    const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES), sb = sa + L * A_BYTES;
+                    if (pass == 0) {
+#pragma unroll
+                        for (int p = 0; p < 4; ++p) {
+                            const uint64_t ad = smem_desc(sa + p * A_BYTES, 128, 256);
+#pragma unroll
+                            for (int q = 0; q < 4 - p; ++q)
+                                tc_mma_i8(tmem + (uint32_t)((p + q) * BN), ad, smem_desc(sb + q * B_BYTES, 128, 256),
+                                          IDESC, (kb > kb0 || p > 0) ? 1u : 0u);
+                        }
+                    } else {
+#pragma unroll
+                        for (int p = 0; p < 8; ++p) {
+                            const uint64_t ad = smem_desc(sa + p * A_BYTES, 128, 256);
+#pragma unroll
+                            for (int q = (p < 4 ? 4 - p : 0); q < 8 - p; ++q)
+                                tc_mma_i8(tmem + (uint32_t)((p + q - 4) * BN), ad,
+                                          smem_desc(sb + q * B_BYTES, 128, 256), IDESC, (kb > kb0 || p > 0) ? 1u : 0u);
+                        }
+                    }
+                    tc_commit(smem_u32(&empty[stage]));
+                    if (++stage == STAGES) { stage = 0; phase ^= 1; }
+                }
+                tc_commit(smem_u32(accf));
+            }
+        }
+    } else {
+        // ---------------- epilogue warps 2..5 ----------------
+        const int quarter = warp & 3;
+        const int64_t row = (int64_t)rb * BM + quarter * 32 + lane;
+        const uint32_t lane_base = tmem + ((uint32_t)(quarter * 32) << 16);
+        const int64_t col0 = (int64_t)nb * BN;
+        // pass L: low = sum_{s<4} S_s 2^{8s}
+        mbar_wait(smem_u32(accf), 0);
+        tc_fence_after();
+#pragma unroll 1
+        for (int j0 = 0; j0 < BN; j0 += 16) {
+            T acc[16];
+#pragma unroll
+            for (int j = 0; j < 16; ++j) acc[j] = 0;
+#pragma unroll
+            for (int s = 0; s < 4; ++s) {
+                uint32_t r[16];
+                tmem_ld16(lane_base + (uint32_t)(s * BN + j0), r);
+#pragma unroll
+                for (int j = 0; j < 16; ++j) acc[j] += (T)r[j] << (8 * s);
+            }
+            if (row < P.M) {
+#pragma unroll
+                for (int j = 0; j < 16; ++j) {
+                    const int64_t col = col0 + j0 + j;
+                    if (col >= P.N) break;
+                    const int64_t o = row * P.N + col;
+                    if (P.mode == 3) atomicAdd((unsigned long long *)(P.partial + (int64_t)party * P.M * P.N + o), acc[j]);
+                    else P.C[P.mode == 2 ? 0 : party][o] = acc[j];
+                }
+            }
+        }
+        tc_fence_before();
+        mbar_arrive(smem_u32(acce));
+        // pass H: high = sum_{s>=4} S_s 2^{8(s-4)} mod 2^32, result = low + high 2^32
+        mbar_wait(smem_u32(accf), 1);
+        tc_fence_after();
+#pragma unroll 1
+        for (int j0 = 0; j0 < BN; j0 += 16) {
+            uint32_t hi[16];
+#pragma unroll
+            for (int j = 0; j < 16; ++j) hi[j] = 0;
+#pragma unroll
+            for (int s = 0; s < 4; ++s) {
+                uint32_t r[16];
+                tmem_ld16(lane_base + (uint32_t)(s * BN + j0), r);
+#pragma unroll
+                for (int j = 0; j < 16; ++j) hi[j] += r[j] << (8 * s);
+            }
+            if (row < P.M) {
+#pragma unroll
+                for (int j = 0; j < 16; ++j) {
+                    const int64_t col = col0 + j0 + j;
+                    if (col >= P.N) break;
+                    const int64_t o = row * P.N + col;
+                    const T h = (T)hi[j] << 32;
+                    switch (P.mode) {
+                    case 0: P.C[party][o] = P.C[party][o] + h; break;
+                    case 1: P.C[party][o] = trunc_share<T>(P.C[party][o] + h + P.Z[party][o], party, P.trunc); break;
+                    case 2: P.C[0][o] = P.C[0][o] + h - P.Z[0][o]; break;
+                    default: atomicAdd((unsigned long long *)(P.partial + (int64_t)party * P.M * P.N + o), h);
+                    }
+                }
+            }
+        }
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 2) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tmem));
+}
+
 template <typename T>
 __global__ void tc_finalize_kernel(const TcParams<T> P, int mode) {
     const int64_t total = P.M * P.N * P.nparty;
@@ -329,7 +516,7 @@ __global__ void tc_finalize_kernel(const TcParams<T> P, int mode) {
 // host side
 // ------------------------------------------------------------------------------------------------
 template <int l> struct Cfg;
-template <> struct Cfg<64> { using T = uint64_t; static constexpr int L = 8, BN = 64, STAGES = 4; static constexpr int MAX_KB = 16384 / BK; };
+template <> struct Cfg<64> { using T = uint64_t; static constexpr int L = 8, BN = 128, STAGES = 3; static constexpr int MAX_KB = 16384 / BK; };
 template <> struct Cfg<32> { using T = uint32_t; static constexpr int L = 4, BN = 128, STAGES = 6; static constexpr int MAX_KB = 1 << 30; };
 
 template <int l>
@@ -386,16 +573,26 @@ static psml_status launch_gemm(TcParams<typename Cfg<l>::T> P, int64_t Mp, int64
         P.mode = 3;
         PSML_CUDA_TRY(cudaMemsetAsync(partial, 0, sizeof(T) * P.M * P.N * P.nparty, s));
     }
-    auto kern = tc_ring_gemm_kernel<T, Cfg<l>::L, BN, Cfg<l>::STAGES>;
-    static bool attr_set = false;
-    if (!attr_set) {
-        PSML_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_bytes<l>()));
-        attr_set = true;
-    }
     dim3 grid((unsigned)(Np / BN), (unsigned)(Mp / BM), (unsigned)(P.nparty * splits));
     {
         ProfScope prof(PROF_TC, s, (double)P.M * P.N * (double)(P.nkb_lo + P.nkb_hi) * BK * P.nparty);
-        kern<<<grid, 128, smem_bytes<l>(), s>>>(P);
+        if constexpr (l == 64) {
+            auto kern = tc_ring_gemm64_v2<Cfg<l>::STAGES>;
+            static bool attr_set = false;
+            if (!attr_set) {
+                PSML_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_bytes<l>()));
+                attr_set = true;
+            }
+            kern<<<grid, 192, smem_bytes<l>(), s>>>(P);
+        } else {
+            auto kern = tc_ring_gemm_kernel<T, Cfg<l>::L, BN, Cfg<l>::STAGES>;
+            static bool attr_set = false;
+            if (!attr_set) {
+                PSML_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_bytes<l>()));
+                attr_set = true;
+            }
+            kern<<<grid, 128, smem_bytes<l>(), s>>>(P);
+        }
         PSML_LAUNCH_CHECK();
     }
     if (splits > 1) {

@@ -64,17 +64,24 @@ struct psml_model_s {
     // activations
     std::vector<psml::Buf> act, z, drelu;  // act[l]: input of layer l (l >= 1 model-owned)
     psml::Buf yhat, delta, tmp;
-    std::vector<psml::DealItem> items;
-    psml::T *ws = nullptr;
+    // Dealer pools, double-buffered: step s consumes pool s % 2, so the dealer of step s + 1 can
+    // run concurrently with the online phase of step s (offline/online pipelining).
+    std::vector<psml::DealItem> items[2];
+    int pool = 0;                      // pool the online phase is reading
+    psml::T *ws = nullptr;             // online workspace
     int64_t ws_words = 0;
+    psml::T *dws = nullptr;            // dealer workspace (split-K partials of Z = U V)
+    int64_t dws_words = 0;
     std::vector<void *> allocs;
-    int64_t dealt_step = -1;
-    bool dealt_full = false;
+    int64_t dealt_step[2] = {-1, -1};
+    bool dealt_full[2] = {false, false};
     bool grads_ready = false;
     uint32_t *step_dev = nullptr;      // device copy of the step number (dealer call ids)
-    cudaGraphExec_t graph = nullptr;   // captured step (psml_model_capture_step)
+    cudaGraphExec_t graph[2] = {nullptr, nullptr};  // captured step(s) (psml_model_capture_step)
     int graph_flags = 0;
     int64_t graph_kernels = 0;
+    cudaStream_t side = nullptr;       // dealer branch inside the pipelined graph
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
 };
 
 namespace psml {
@@ -98,7 +105,7 @@ static psml_status balloc(psml_model_s *m, Buf &b, int64_t n) {
 }
 
 static DealItem *find_item(psml_model_s *m, int layer, int op, int slot) {
-    for (auto &it : m->items)
+    for (auto &it : m->items[m->pool])
         if (it.layer == layer && it.op == op && it.slot == slot) return &it;
     return nullptr;
 }
@@ -106,17 +113,17 @@ static DealItem *find_item(psml_model_s *m, int layer, int op, int slot) {
 static void add_matrix(psml_model_s *m, int layer, int op, int64_t M, int64_t K, int64_t N, bool fwd) {
     DealItem it;
     it.kind = IT_MATRIX; it.layer = layer; it.op = op; it.slot = 0; it.M = M; it.K = K; it.N = N; it.fwd = fwd;
-    m->items.push_back(it);
+    m->items[0].push_back(it);
 }
 static void add_had(psml_model_s *m, int layer, int slot, int64_t n, bool fwd) {
     DealItem it;
     it.kind = IT_HAD; it.layer = layer; it.op = OP_HADAMARD; it.slot = slot; it.n = n; it.fwd = fwd;
-    m->items.push_back(it);
+    m->items[0].push_back(it);
 }
 static void add_msb(psml_model_s *m, int layer, int op, int64_t n, bool fwd) {
     DealItem it;
     it.kind = IT_MSB; it.layer = layer; it.op = op; it.slot = 0; it.n = n; it.fwd = fwd;
-    m->items.push_back(it);
+    m->items[0].push_back(it);
 }
 
 static bool is_eq9_out(const psml_model_s *m) { return m->d.kind != PSML_LINREG; }
@@ -130,7 +137,7 @@ static void plan_items(psml_model_s *m) {
         DealItem cf;
         cf.kind = IT_CONV_FWD; cf.layer = 0; cf.op = OP_FWD; cf.slot = 0;
         cf.M = rows; cf.K = kk; cf.N = m->cols[0]; cf.fwd = true;
-        m->items.push_back(cf);
+        m->items[0].push_back(cf);
         add_msb(m, 0, OP_RELU_MSB, B * h1, true);
         add_had(m, 0, 0, B * h1, true);
         add_matrix(m, 1, OP_FWD, B, h1, hid, true);
@@ -148,7 +155,7 @@ static void plan_items(psml_model_s *m) {
         DealItem cg;
         cg.kind = IT_CONV_GW; cg.layer = 0; cg.op = OP_GRADW; cg.slot = 0;
         cg.M = kk; cg.K = rows; cg.N = m->cols[0]; cg.fwd = false;
-        m->items.push_back(cg);
+        m->items[0].push_back(cg);
         return;
     }
     const int nl = m->nl;
@@ -172,9 +179,9 @@ static void plan_items(psml_model_s *m) {
     }
 }
 
-static psml_status alloc_items(psml_model_s *m) {
+static psml_status alloc_items(psml_model_s *m, std::vector<DealItem> &items) {
     const psml_ring ring = m->ctx->ring;
-    for (auto &it : m->items) {
+    for (auto &it : items) {
         switch (it.kind) {
         case IT_MATRIX:
             PSML_TRY(balloc(m, it.U, it.M * it.K));
@@ -204,7 +211,7 @@ static psml_status alloc_items(psml_model_s *m) {
 
 static int64_t ws_need(psml_model_s *m) {
     int64_t w = 0;
-    for (auto &it : m->items) {
+    for (auto &it : m->items[0]) {
         switch (it.kind) {
         case IT_MATRIX: w = std::max(w, beaver_ws_words<T>(it.M, it.K, it.N)); break;
         case IT_CONV_FWD: w = std::max(w, conv_ws_words<T>(m->B, m->g, 0, it.N)); break;
@@ -213,8 +220,12 @@ static int64_t ws_need(psml_model_s *m) {
         case IT_MSB: w = std::max(w, msb_ws_words<T>(it.n)); break;
         }
     }
-    // dealer: conv Z GEMM split-K partials + plain triplet partials
-    for (auto &it : m->items)
+    return w;
+}
+
+static int64_t dws_need(psml_model_s *m) {
+    int64_t w = 1;   // dealer: split-K partials of the Z = U V GEMMs
+    for (auto &it : m->items[0])
         if (it.kind != IT_HAD && it.kind != IT_MSB) w = std::max(w, it.M * it.N);
     return w;
 }
@@ -222,53 +233,63 @@ static int64_t ws_need(psml_model_s *m) {
 // ------------------------------------------------------------------------------------------------
 // dealer (offline phase)
 // ------------------------------------------------------------------------------------------------
+// PRG part of a matrix / conv triplet: U_0, U_1 (n_u), V_0, V_1 (K x N), Z_0 (M x N)
+static psml_status deal_prg(psml_model_s *m, DealItem &it, uint64_t cid, cudaStream_t s) {
+    const uint64_t seed = m->d.dealer_seed;
+    ProfScope prof(PROF_DEALER, s, (double)sizeof(T) * (2 * it.U.n + 2 * it.V.n + it.Z.n));
+    dealer_pair_kernel<T><<<grid_for(it.U.n / 8 + 1, 256), 256, 0, s>>>(
+        make_key(seed, TAG_U0, cid, m->step_dev), make_key(seed, TAG_U1, cid, m->step_dev), it.U.n, it.U.p[0],
+        it.U.p[1], nullptr);
+    PSML_LAUNCH_CHECK();
+    dealer_pair_kernel<T><<<grid_for(it.V.n / 8 + 1, 256), 256, 0, s>>>(
+        make_key(seed, TAG_V0, cid, m->step_dev), make_key(seed, TAG_V1, cid, m->step_dev), it.V.n, it.V.p[0],
+        it.V.p[1], nullptr);
+    PSML_LAUNCH_CHECK();
+    prg_kernel<T, 0><<<grid_for(it.Z.n / 8 + 2, 256), 256, 0, s>>>(make_key(seed, TAG_Z0, cid, m->step_dev), 0, it.Z.n,
+                                                                     it.Z.p[0], nullptr, nullptr);
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
 static psml_status deal_item(psml_model_s *m, DealItem &it, uint32_t step, cudaStream_t s) {
     const uint64_t seed = m->d.dealer_seed;
-    ProfScope prof(PROF_DEALER, s, (double)sizeof(T) * 2 * (it.U.n + it.V.n + it.Z.n + it.mat.n));
     const uint64_t cid = call_id(m->d.pair_id, step, it.layer, it.op, it.slot);
     switch (it.kind) {
     case IT_MATRIX: {
-        dealer_pair_kernel<T><<<grid_for(it.M * it.K / 8 + 1, 256), 256, 0, s>>>(
-            make_key(seed, TAG_U0, cid, m->step_dev), make_key(seed, TAG_U1, cid, m->step_dev), it.M * it.K, it.U.p[0], it.U.p[1], nullptr);
-        PSML_LAUNCH_CHECK();
-        dealer_pair_kernel<T><<<grid_for(it.K * it.N / 8 + 1, 256), 256, 0, s>>>(
-            make_key(seed, TAG_V0, cid, m->step_dev), make_key(seed, TAG_V1, cid, m->step_dev), it.K * it.N, it.V.p[0], it.V.p[1], nullptr);
-        PSML_LAUNCH_CHECK();
-        prg_kernel<T, 0><<<grid_for(it.M * it.N / 8 + 2, 256), 256, 0, s>>>(make_key(seed, TAG_Z0, cid, m->step_dev), 0,
-                                                                            it.M * it.N, it.Z.p[0], nullptr, nullptr);
-        PSML_LAUNCH_CHECK();
-        DealerOps<T> ops;
+        PSML_TRY(deal_prg(m, it, cid, s));
+        DealerOps<T> ops;   // Z_1 = (U_0 + U_1)(V_0 + V_1) - Z_0
         ops.U0 = it.U.p[0]; ops.U1 = it.U.p[1]; ops.V0 = it.V.p[0]; ops.V1 = it.V.p[1];
         ops.Z0 = it.Z.p[0]; ops.Z1 = it.Z.p[1];
         ops.M = it.M; ops.N = it.N; ops.Kext = it.K;
-        return launch_ring_gemm<T, DealerOps<T>>(ops, m->ws, m->ws_words, s, m->ctx->sm_count);
+        return launch_ring_gemm<T, DealerOps<T>>(ops, m->dws, m->dws_words, s, m->ctx->sm_count);
     }
     case IT_CONV_FWD:
     case IT_CONV_GW: {
-        const int64_t nin = it.U.n;
-        dealer_pair_kernel<T><<<grid_for(nin / 8 + 1, 256), 256, 0, s>>>(
-            make_key(seed, TAG_U0, cid, m->step_dev), make_key(seed, TAG_U1, cid, m->step_dev), nin, it.U.p[0], it.U.p[1], nullptr);
-        PSML_LAUNCH_CHECK();
-        dealer_pair_kernel<T><<<grid_for(it.K * it.N / 8 + 1, 256), 256, 0, s>>>(
-            make_key(seed, TAG_V0, cid, m->step_dev), make_key(seed, TAG_V1, cid, m->step_dev), it.K * it.N, it.V.p[0], it.V.p[1], nullptr);
-        PSML_LAUNCH_CHECK();
-        prg_kernel<T, 0><<<grid_for(it.M * it.N / 8 + 2, 256), 256, 0, s>>>(make_key(seed, TAG_Z0, cid, m->step_dev), 0,
-                                                                            it.M * it.N, it.Z.p[0], nullptr, nullptr);
-        PSML_LAUNCH_CHECK();
-        ConvDealerOps<T> ops;
+        PSML_TRY(deal_prg(m, it, cid, s));
+        ConvDealerOps<T> ops;   // Z_1 = im2col(U_0 + U_1) (^T) (V_0 + V_1) - Z_0
         ops.U0 = it.U.p[0]; ops.U1 = it.U.p[1]; ops.V0 = it.V.p[0]; ops.V1 = it.V.p[1];
         ops.Z0 = it.Z.p[0]; ops.Z1 = it.Z.p[1];
         ops.g = m->g; ops.M = it.M; ops.N = it.N; ops.Kext = it.K; ops.transposed = it.kind == IT_CONV_GW;
-        return launch_ring_gemm<T, ConvDealerOps<T>>(ops, m->ws, m->ws_words, s, m->ctx->sm_count);
+        return launch_ring_gemm<T, ConvDealerOps<T>>(ops, m->dws, m->dws_words, s, m->ctx->sm_count);
     }
     case IT_HAD: {
+        ProfScope prof(PROF_DEALER, s, (double)sizeof(T) * 6 * it.n);
         void *U[2] = {it.U.p[0], it.U.p[1]}, *V[2] = {it.V.p[0], it.V.p[1]}, *Z[2] = {it.Z.p[0], it.Z.p[1]};
         return hadamard_triplet_launch<T>(seed, cid, it.n, U, V, Z, s, m->step_dev);
     }
     case IT_MSB: {
+        ProfScope prof(PROF_DEALER, s, (double)sizeof(T) * 2 * it.mat.n);
         void *mt[2] = {it.mat.p[0], it.mat.p[1]};
         return msb_dealer_launch<T>(seed, cid, it.n, mt, s, m->step_dev);
     }
+    }
+    return PSML_OK;
+}
+
+static psml_status deal_pool(psml_model_s *m, int pool, uint32_t step, bool infer_only, cudaStream_t s) {
+    for (auto &it : m->items[pool]) {
+        if (infer_only && !it.fwd) continue;
+        PSML_TRY(deal_item(m, it, step, s));
     }
     return PSML_OK;
 }
@@ -467,7 +488,14 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
     PSML_TRY(balloc(mp, m->delta, B * maxw));
     PSML_TRY(balloc(mp, m->tmp, B * maxw));
     plan_items(mp);
-    PSML_TRY(alloc_items(mp));
+    m->items[1] = m->items[0];
+    PSML_TRY(alloc_items(mp, m->items[0]));
+    PSML_TRY(alloc_items(mp, m->items[1]));
+    m->dws_words = dws_need(mp);
+    PSML_TRY(dalloc(mp, &m->dws, m->dws_words));
+    PSML_CUDA_TRY(cudaStreamCreateWithFlags(&m->side, cudaStreamNonBlocking));
+    PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_fork, cudaEventDisableTiming));
+    PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_join, cudaEventDisableTiming));
     {
         T *sd = nullptr;
         PSML_TRY(dalloc(mp, &sd, 1));
@@ -482,7 +510,11 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
 psml_status psml_model_destroy(psml_model model) {
     if (!model) return PSML_OK;
     cudaDeviceSynchronize();
-    if (model->graph) cudaGraphExecDestroy(model->graph);
+    for (int g = 0; g < 2; ++g)
+        if (model->graph[g]) cudaGraphExecDestroy(model->graph[g]);
+    if (model->side) cudaStreamDestroy(model->side);
+    if (model->ev_fork) cudaEventDestroy(model->ev_fork);
+    if (model->ev_join) cudaEventDestroy(model->ev_join);
     for (void *p : model->allocs) cudaFree(p);
     delete model;
     return PSML_OK;
@@ -521,14 +553,12 @@ psml_status psml_model_get_master(psml_model m, int32_t layer, void *const Wm[2]
 psml_status psml_model_deal(psml_model m, uint32_t step_id, int32_t infer_only, psml_stream stream) {
     if (!m) return fail(PSML_ERR_INVALID, "model is null");
     cudaStream_t s = (cudaStream_t)stream;
+    const int pool = (int)(step_id & 1);
     set_word_kernel<<<1, 1, 0, s>>>(m->step_dev, step_id);
     PSML_LAUNCH_CHECK();
-    for (auto &it : m->items) {
-        if (infer_only && !it.fwd) continue;
-        PSML_TRY(deal_item(m, it, step_id, s));
-    }
-    m->dealt_step = step_id;
-    m->dealt_full = !infer_only;
+    PSML_TRY(deal_pool(m, pool, step_id, infer_only != 0, s));
+    m->dealt_step[pool] = step_id;
+    m->dealt_full[pool] = !infer_only;
     return PSML_OK;
 }
 
@@ -536,9 +566,11 @@ psml_status psml_train_forward_backward(psml_model m, const void *const X[2], co
                                         psml_stream stream) {
     if (!m || !X || !Y) return fail(PSML_ERR_INVALID, "null argument");
     PSML_TRY(check_ptrs({X[0], X[1], Y[0], Y[1]}));
-    if (m->dealt_step != (int64_t)step_id || !m->dealt_full)
+    const int pool = (int)(step_id & 1);
+    if (m->dealt_step[pool] != (int64_t)step_id || !m->dealt_full[pool])
         return fail(PSML_ERR_STATE, "psml_model_deal(step_id, infer_only=0) must precede the step");
     cudaStream_t s = (cudaStream_t)stream;
+    m->pool = pool;
     PSML_TRY(forward(m, (const T *const *)X, (const T *const *)Y, nullptr, s));
     PSML_TRY(backward(m, s));
     m->grads_ready = true;
@@ -587,32 +619,34 @@ psml_status psml_secure_train_step(psml_model m, const void *const X[2], const v
     return psml_train_apply_update(m, 0, stream);
 }
 
-psml_status psml_model_capture_step(psml_model m, const void *const X[2], const void *const Y[2], int32_t flags,
-                                   psml_stream stream) {
-    if (!m || !X || !Y) return fail(PSML_ERR_INVALID, "null argument");
-    PSML_TRY(check_ptrs({X[0], X[1], Y[0], Y[1]}));
-    if (flags & ~3) return fail(PSML_ERR_INVALID, "flags: bit 0 = with dealer, bit 1 = with update");
-    cudaStream_t s = (cudaStream_t)stream;
-    if (s == nullptr) return fail(PSML_ERR_INVALID, "capture needs a non-default stream");
-    if (m->graph) {
-        cudaGraphExecDestroy(m->graph);
-        m->graph = nullptr;
-    }
-    const int prof = g_prof_cls.exchange(-1);   // no profiling events inside the graph
+// One captured step for online pool `pool`.  Non-pipelined: [dealer(pool)] -> online -> [update].
+// Pipelined: online(pool) -> [update] on `s`, concurrently dealer(1 - pool) for the NEXT step on the
+// side stream (fork/join inside the capture), reading the step word = step + 1.
+static psml_status capture_one(psml_model_s *m, int pool, const T *const X[2], const T *const Y[2], int flags,
+                               cudaStream_t s, cudaGraphExec_t *out, int64_t *kernels) {
+    const bool pipelined = (flags & 4) != 0;
     PSML_CUDA_TRY(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
     psml_status st = PSML_OK;
-    if (flags & 1)
-        for (auto &it : m->items)
-            if (st == PSML_OK) st = deal_item(m, it, 0, s);
-    if (st == PSML_OK) st = forward(m, (const T *const *)X, (const T *const *)Y, nullptr, s);
+    if (pipelined) {
+        if (cudaEventRecord(m->ev_fork, s) != cudaSuccess || cudaStreamWaitEvent(m->side, m->ev_fork, 0) != cudaSuccess)
+            st = fail(PSML_ERR_CUDA, "graph fork failed");
+        if (st == PSML_OK) st = deal_pool(m, 1 - pool, 0, false, m->side);
+        if (st == PSML_OK && cudaEventRecord(m->ev_join, m->side) != cudaSuccess)
+            st = fail(PSML_ERR_CUDA, "graph join record failed");
+    } else if (flags & 1) {
+        st = deal_pool(m, pool, 0, false, s);
+    }
+    m->pool = pool;
+    if (st == PSML_OK) st = forward(m, X, Y, nullptr, s);
     if (st == PSML_OK) st = backward(m, s);
     if (st == PSML_OK && (flags & 2)) {
         m->grads_ready = true;
-        st = psml_train_apply_update(m, 0, stream);
+        st = psml_train_apply_update(m, 0, (psml_stream)s);
     }
+    if (pipelined && st == PSML_OK && cudaStreamWaitEvent(s, m->ev_join, 0) != cudaSuccess)
+        st = fail(PSML_ERR_CUDA, "graph join failed");
     cudaGraph_t g = nullptr;
     cudaError_t e = cudaStreamEndCapture(s, &g);
-    g_prof_cls.store(prof);
     if (st != PSML_OK) {
         if (g) cudaGraphDestroy(g);
         return st;
@@ -622,14 +656,37 @@ psml_status psml_model_capture_step(psml_model m, const void *const X[2], const 
     cudaGraphGetNodes(g, nullptr, &nn);
     std::vector<cudaGraphNode_t> nodes(nn);
     if (nn) cudaGraphGetNodes(g, nodes.data(), &nn);
-    m->graph_kernels = 0;
+    *kernels = 0;
     for (auto nd : nodes) {
         cudaGraphNodeType t;
-        if (cudaGraphNodeGetType(nd, &t) == cudaSuccess && t == cudaGraphNodeTypeKernel) ++m->graph_kernels;
+        if (cudaGraphNodeGetType(nd, &t) == cudaSuccess && t == cudaGraphNodeTypeKernel) ++*kernels;
     }
-    e = cudaGraphInstantiate(&m->graph, g, 0);
+    e = cudaGraphInstantiate(out, g, 0);
     cudaGraphDestroy(g);
     if (e != cudaSuccess) return fail(PSML_ERR_CUDA, std::string("graph instantiate: ") + cudaGetErrorString(e));
+    return PSML_OK;
+}
+
+psml_status psml_model_capture_step(psml_model m, const void *const X[2], const void *const Y[2], int32_t flags,
+                                   psml_stream stream) {
+    if (!m || !X || !Y) return fail(PSML_ERR_INVALID, "null argument");
+    PSML_TRY(check_ptrs({X[0], X[1], Y[0], Y[1]}));
+    if (flags & ~7) return fail(PSML_ERR_INVALID, "flags: bit 0 dealer, bit 1 update, bit 2 pipelined dealer");
+    cudaStream_t s = (cudaStream_t)stream;
+    if (s == nullptr) return fail(PSML_ERR_INVALID, "capture needs a non-default stream");
+    for (int g = 0; g < 2; ++g)
+        if (m->graph[g]) {
+            cudaGraphExecDestroy(m->graph[g]);
+            m->graph[g] = nullptr;
+        }
+    const int prof = g_prof_cls.exchange(-1);   // no profiling events inside the graphs
+    psml_status st = PSML_OK;
+    const int ngraphs = (flags & 4) ? 2 : 1;
+    for (int g = 0; g < ngraphs && st == PSML_OK; ++g)
+        st = capture_one(m, (flags & 4) ? g : 0, (const T *const *)X, (const T *const *)Y, flags, s, &m->graph[g],
+                         &m->graph_kernels);
+    g_prof_cls.store(prof);
+    if (st != PSML_OK) return st;
     m->graph_flags = flags;
     return PSML_OK;
 }
@@ -642,13 +699,23 @@ psml_status psml_model_graph_nodes(psml_model m, int64_t *n) {
 
 psml_status psml_model_step_graph(psml_model m, uint32_t step_id, psml_stream stream) {
     if (!m) return fail(PSML_ERR_INVALID, "model is null");
-    if (!m->graph) return fail(PSML_ERR_STATE, "no captured step: call psml_model_capture_step first");
+    if (!m->graph[0]) return fail(PSML_ERR_STATE, "no captured step: call psml_model_capture_step first");
     cudaStream_t s = (cudaStream_t)stream;
-    set_word_kernel<<<1, 1, 0, s>>>(m->step_dev, step_id);
+    const bool pipelined = (m->graph_flags & 4) != 0;
+    const int pool = pipelined ? (int)(step_id & 1) : 0;
+    if (pipelined && (m->dealt_step[pool] != (int64_t)step_id || !m->dealt_full[pool]))
+        return fail(PSML_ERR_STATE, "pipelined graph: psml_model_deal(step_id) must have filled this step's pool");
+    set_word_kernel<<<1, 1, 0, s>>>(m->step_dev, pipelined ? step_id + 1 : step_id);
     PSML_LAUNCH_CHECK();
-    PSML_CUDA_TRY(cudaGraphLaunch(m->graph, s));
+    PSML_CUDA_TRY(cudaGraphLaunch(m->graph[pipelined ? pool : 0], s));
     g_launches.fetch_add((uint64_t)m->graph_kernels);   // the graph's kernels are our launches
-    if (m->graph_flags & 1) { m->dealt_step = step_id; m->dealt_full = true; }
+    if (pipelined) {
+        m->dealt_step[1 - pool] = (int64_t)step_id + 1;
+        m->dealt_full[1 - pool] = true;
+    } else if (m->graph_flags & 1) {
+        m->dealt_step[0] = step_id;
+        m->dealt_full[0] = true;
+    }
     m->grads_ready = !(m->graph_flags & 2);
     return PSML_OK;
 }
@@ -657,7 +724,10 @@ psml_status psml_secure_infer(psml_model m, const void *const X[2], uint32_t ste
                               psml_stream stream) {
     if (!m || !X || !Yhat) return fail(PSML_ERR_INVALID, "null argument");
     PSML_TRY(check_ptrs({X[0], X[1], Yhat[0], Yhat[1]}));
-    if (m->dealt_step != (int64_t)step_id) return fail(PSML_ERR_STATE, "psml_model_deal(step_id) must precede inference");
+    const int pool = (int)(step_id & 1);
+    if (m->dealt_step[pool] != (int64_t)step_id)
+        return fail(PSML_ERR_STATE, "psml_model_deal(step_id) must precede inference");
+    m->pool = pool;
     return forward(m, (const T *const *)X, nullptr, (T *const *)Yhat, (cudaStream_t)stream);
 }
 

@@ -426,9 +426,10 @@ class Model:
     def apply_update(self, extra_shift=0, stream=None):
         _call("psml_train_apply_update", self.handle, extra_shift, _stream(stream))
 
-    def capture_step(self, X, Y, with_deal=True, with_update=True, stream=None):
-        """Capture one step into a CUDA graph reading the fixed share buffers X, Y."""
-        flags = (1 if with_deal else 0) | (2 if with_update else 0)
+    def capture_step(self, X, Y, with_deal=True, with_update=True, pipelined=False, stream=None):
+        """Capture one step into a CUDA graph reading the fixed share buffers X, Y (pipelined:
+        the dealer of step s + 1 overlaps the online phase of step s)."""
+        flags = (1 if with_deal else 0) | (2 if with_update else 0) | (4 if pipelined else 0)
         _call("psml_model_capture_step", self.handle, _pair(X), _pair(Y), flags, _stream(stream))
 
     def graph_nodes(self):

@@ -62,9 +62,10 @@ class SecureTrainer:
         return Xs, Ys
 
     # --- steps --------------------------------------------------------------------------------
-    def capture(self, with_update=True):
-        """Capture deal + online step (+ update) into a CUDA graph on a side stream; the batch is
-        shared into fixed buffers before each replay (graph_step)."""
+    def capture(self, with_update=True, pipelined=True):
+        """Capture deal + online step (+ update) into CUDA graph(s) on a side stream; the batch is
+        shared into fixed buffers before each replay (graph_step).  pipelined: the dealer of the
+        next step runs concurrently with the online phase of this one (double-buffered pools)."""
         d_in = self.model.layer_shape(0)[0] if self.task != "cnn" else 3 * 32 * 32
         self.Xbuf = psml.empty_pair((self.batch, d_in), 64)
         self.Ybuf = psml.empty_pair((self.batch, self.out_dim), 64)
@@ -74,9 +75,11 @@ class SecureTrainer:
         self.gstream.wait_stream(torch.cuda.current_stream())
         with torch.cuda.stream(self.gstream):
             self.model.capture_step(self.Xbuf, self.Ybuf, with_deal=True, with_update=with_update,
-                                    stream=self.gstream)
+                                    pipelined=pipelined, stream=self.gstream)
         torch.cuda.current_stream().wait_stream(self.gstream)
         self.graph_update = with_update
+        self.pipelined = pipelined
+        self._next_dealt = None
 
     def graph_kernel_nodes(self):
         return self.model.graph_nodes()
@@ -87,7 +90,10 @@ class SecureTrainer:
         y = psml.encode(self.ring, torch.as_tensor(Y, dtype=torch.float64))
         psml.share(self.ring, SHARE_SEED, call_id(self.pair_id, step, 0, OP_SHARE, 0), x, out=self.Xbuf)
         psml.share(self.ring, SHARE_SEED, call_id(self.pair_id, step, 0, OP_SHARE, 1), y, out=self.Ybuf)
+        if self.pipelined and self._next_dealt != step:
+            self.model.deal(step)          # prime the pipeline (first step or a jump in step ids)
         self.model.step_graph(step)
+        self._next_dealt = step + 1
 
     def deal(self, step, infer_only=False):
         self.model.deal(step, infer_only=infer_only)

@@ -79,8 +79,9 @@ def test_one_epoch_within_2pow_minus12_of_fp64(T, task, tol_log2):
     tr.close()
 
 
-@pytest.mark.parametrize("task,steps", [("mlp", 3), ("logreg", 2)])
-def test_graph_replay_bitexact_vs_oracle(T, task, steps):
+@pytest.mark.parametrize("task,steps,pipelined", [("mlp", 3, True), ("mlp", 2, False),
+                                                  ("logreg", 2, True), ("cnn", 1, True)])
+def test_graph_replay_bitexact_vs_oracle(T, task, steps, pipelined):
     """The captured CUDA graph (dealer + online step + update, step id from a device word)
     reproduces the oracle's shares exactly for successive step ids."""
     Wi = synth.init_weights(task)
@@ -89,7 +90,7 @@ def test_graph_replay_bitexact_vs_oracle(T, task, steps):
     X, Y = synth.batch(task, 0)
     tr.step(torch.from_numpy(X), torch.from_numpy(Y), 0)      # eager warm-up step 0
     OP.train_step(om, X, Y, 0)
-    tr.capture()
+    tr.capture(pipelined=pipelined)
     for s in range(1, steps + 1):
         X, Y = synth.batch(task, s)
         tr.graph_step(torch.from_numpy(X), torch.from_numpy(Y), s)
