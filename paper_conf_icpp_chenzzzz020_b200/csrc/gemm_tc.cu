@@ -193,6 +193,43 @@ struct TcParams {
     T *partial;        // mode 3: nparty x M x N
 };
 
+// Epilogue chunk: thread `lane` holds 16 consecutive columns of row row0 + lane (the TMEM 32x32b
+// fragment).  Transpose through a per-warp smem tile (32 x 17 words, padded) so that each store /
+// read-modify-write instruction covers two 128-byte row segments instead of 32 scattered words.
+// phase 0: v = low part (or the whole result in single-pass kernels); phase 1: v = high part.
+template <typename T>
+__device__ __forceinline__ void epi_chunk(T *st, const T v[16], int lane, int64_t row0, int64_t col0,
+                                          const TcParams<T> &P, int party, int phase, bool two_pass) {
+#pragma unroll
+    for (int j = 0; j < 16; ++j) st[lane * 17 + j] = v[j];
+    __syncwarp();
+    const int c = lane & 15, rs = lane >> 4;
+    const int64_t col = col0 + c;
+#pragma unroll 4
+    for (int r = 0; r < 16; ++r) {
+        const int rl = 2 * r + rs;
+        const int64_t row = row0 + rl;
+        if (row >= P.M || col >= P.N) continue;
+        const T x = st[rl * 17 + c];
+        const int64_t o = row * P.N + col;
+        if (P.mode == 3) {
+            T *dst = P.partial + (int64_t)party * P.M * P.N + o;
+            if (sizeof(T) == 8) atomicAdd((unsigned long long *)dst, (unsigned long long)x);
+            else atomicAdd((unsigned int *)dst, (unsigned int)x);
+            continue;
+        }
+        T *C = P.C[P.mode == 2 ? 0 : party];
+        if (two_pass && phase == 0) { C[o] = x; continue; }
+        const T acc = two_pass ? (T)(C[o] + x) : x;
+        switch (P.mode) {
+        case 0: C[o] = acc; break;
+        case 1: C[o] = trunc_share<T>(acc + P.Z[party][o], party, P.trunc); break;
+        default: C[o] = acc - P.Z[0][o]; break;
+        }
+    }
+    __syncwarp();
+}
+
 template <typename T, int L, int BN, int STAGES>
 __global__ void __launch_bounds__(128, 1) tc_ring_gemm_kernel(const TcParams<T> P) {
     extern __shared__ __align__(1024) uint8_t smem[];
@@ -276,8 +313,9 @@ __global__ void __launch_bounds__(128, 1) tc_ring_gemm_kernel(const TcParams<T> 
     // ---------------- epilogue: sum_s S_s 2^{8s} mod 2^l, + Z, trunc, store ----------------
     mbar_wait(smem_u32(accum), 0);
     tc_fence_after();
-    const int64_t row = (int64_t)rb * BM + warp * 32 + lane;
+    const int64_t row0 = (int64_t)rb * BM + warp * 32;
     const uint32_t lane_base = tmem + ((uint32_t)(warp * 32) << 16);
+    T *st = (T *)smem + warp * 32 * 17;   // pipeline smem is idle now: reuse it for staging
 #pragma unroll 1
     for (int j0 = 0; j0 < BN; j0 += 16) {
         T acc[16];
@@ -290,25 +328,7 @@ __global__ void __launch_bounds__(128, 1) tc_ring_gemm_kernel(const TcParams<T> 
 #pragma unroll
             for (int j = 0; j < 16; ++j) acc[j] += (T)r[j] << (8 * s);
         }
-        if (row < P.M) {
-            const int64_t col0 = (int64_t)nb * BN + j0;
-#pragma unroll
-            for (int j = 0; j < 16; ++j) {
-                const int64_t col = col0 + j;
-                if (col >= P.N) break;
-                const int64_t o = row * P.N + col;
-                switch (P.mode) {
-                case 0: P.C[party][o] = acc[j]; break;
-                case 1: P.C[party][o] = trunc_share<T>(acc[j] + P.Z[party][o], party, P.trunc); break;
-                case 2: P.C[0][o] = acc[j] - P.Z[0][o]; break;
-                default: {
-                    T *dst = P.partial + (int64_t)party * P.M * P.N + o;
-                    if (sizeof(T) == 8) atomicAdd((unsigned long long *)dst, (unsigned long long)acc[j]);
-                    else atomicAdd((unsigned int *)dst, (unsigned int)acc[j]);
-                }
-                }
-            }
-        }
+        epi_chunk<T>(st, acc, lane, row0, (int64_t)nb * BN + j0, P, party, 0, false);
     }
     tc_fence_before();
     __syncthreads();
@@ -430,6 +450,8 @@ __global__ void __launch_bounds__(192, 1) tc_ring_gemm64_v2(const TcParams<uint6
         }
     } else {
         // ---------------- epilogue warps 2..5 ----------------
+        // Direct per-row stores: staging through smem here would compete with the tensor core's
+        // smem reads of pass H, which this epilogue overlaps (measured slower).
         const int quarter = warp & 3;
         const int64_t row = (int64_t)rb * BM + quarter * 32 + lane;
         const uint32_t lane_base = tmem + ((uint32_t)(quarter * 32) << 16);
@@ -449,6 +471,10 @@ __global__ void __launch_bounds__(192, 1) tc_ring_gemm64_v2(const TcParams<uint6
 #pragma unroll
                 for (int j = 0; j < 16; ++j) acc[j] += (T)r[j] << (8 * s);
             }
+            if (j0 == BN - 16) {   // TMEM fully read: pass H may start before this last store
+                tc_fence_before();
+                mbar_arrive(smem_u32(acce));
+            }
             if (row < P.M) {
 #pragma unroll
                 for (int j = 0; j < 16; ++j) {
@@ -460,8 +486,6 @@ __global__ void __launch_bounds__(192, 1) tc_ring_gemm64_v2(const TcParams<uint6
                 }
             }
         }
-        tc_fence_before();
-        mbar_arrive(smem_u32(acce));
         // pass H: high = sum_{s>=4} S_s 2^{8(s-4)} mod 2^32, result = low + high 2^32
         mbar_wait(smem_u32(accf), 1);
         tc_fence_after();
