@@ -135,6 +135,7 @@ def bench_ours(args):
 
     import synth
     from paper_conf_icpp_chenzzzz020_b200 import build, psml
+    from paper_conf_icpp_chenzzzz020_b200.parallel import dp_update_shift, ring_allreduce_
     from paper_conf_icpp_chenzzzz020_b200.train import SecureTrainer
 
     build.build()
@@ -159,8 +160,8 @@ def bench_ours(args):
         # online step [+ update]); data parallel: NCCL all-reduce of gradient shares + update
         tr.graph_step(X, Y, s)
         if world > 1:
-            dist.all_reduce(tr.grad_tensor(), op=dist.ReduceOp.SUM)
-            tr.model.apply_update(extra_shift=int(round(np.log2(world))))
+            ring_allreduce_(tr.grad_tensor())
+            tr.model.apply_update(extra_shift=dp_update_shift(world))
 
     def one_step(s, X, Y, online_only=False, shares=None):
         if online_only:

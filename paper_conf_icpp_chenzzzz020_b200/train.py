@@ -13,11 +13,10 @@ Data parallelism: one co-resident pair per GPU, each on 
 the untruncated weight-gradient shares are summed across pairs with an all-reduce (uint64 ring
 addition = int64 two's-complement addition), then every pair applies the same update.
 """
-import math
-
 import torch
 
 from . import psml
+from .parallel import dp_update_shift, ring_allreduce_
 
 DATA_SEED = 0x50534D4C
 SHARE_SEED = DATA_SEED + 1
@@ -114,13 +113,8 @@ class SecureTrainer:
             self.model.deal(step)
         self.model.forward_backward(Xs, Ys, step)
         world = dist.get_world_size(group) if dist.is_initialized() else 1
-        if world > 1:
-            g = self.grad_tensor()
-            dist.all_reduce(g, op=dist.ReduceOp.SUM, group=group)
-        extra = int(round(math.log2(world)))
-        if (1 << extra) != world:
-            raise ValueError("data-parallel pair count must be a power of two (R16)")
-        self.model.apply_update(extra_shift=extra)
+        ring_allreduce_(self.grad_tensor(), group)
+        self.model.apply_update(extra_shift=dp_update_shift(world))
 
     def last_yhat(self):
         """Prediction shares of the last step as two uint64 views of model-owned memory."""
