@@ -279,6 +279,71 @@ ring_gemm_tiled(Ops ops, int64_t k_per_split, T *__restrict__ partial) {
 }
 
 // ---------------------------------------------------------------------------------------------
+// small-output kernel: 16 x 16 output tile per 256-thread CTA (one output per thread), K in
+// chunks of 64 staged in smem with the next chunk prefetched into registers.  For the MLP's
+// 128 x 128 products this gives 64-128 CTAs without split-K, i.e. ~K'/64 memory round trips
+// instead of the 64 x 64 tile's K'/16 at ~2 warps per SM.
+// ---------------------------------------------------------------------------------------------
+template <typename T, class Ops>
+__global__ void __launch_bounds__(256) ring_gemm_small(Ops ops, int64_t k_per_split, T *__restrict__ partial) {
+    constexpr int BM = 16, BN = 16, BK = 64;
+    __shared__ T As[2][BM][BK + 1];
+    __shared__ T Bs[2][BK][BN];
+    const int p = blockIdx.z % Ops::nparty;
+    const int split = blockIdx.z / Ops::nparty;
+    const int64_t m0 = (int64_t)blockIdx.y * BM, n0 = (int64_t)blockIdx.x * BN;
+    const int64_t kbeg = (int64_t)split * k_per_split;
+    const int64_t kend = min(ops.Kext, kbeg + k_per_split);
+    const int tid = threadIdx.x;
+    const int tx = tid & 15, ty = tid >> 4;
+    T ra[4], rb[4];
+    auto load = [&](int64_t k0) {
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+            const int idx = tid + t * 256;
+            const int mm = idx >> 6, kk = idx & 63;          // A: 16 x 64, coalesced along k
+            const int64_t m = m0 + mm, k = k0 + kk;
+            ra[t] = (m < ops.M && k < kend) ? ops.a(p, m, k) : (T)0;
+            const int kb = idx >> 4, nn = idx & 15;          // B: 64 x 16, coalesced along n
+            const int64_t k2 = k0 + kb, n = n0 + nn;
+            rb[t] = (n < ops.N && k2 < kend) ? ops.b(p, k2, n) : (T)0;
+        }
+    };
+    auto stash = [&](int buf) {
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+            const int idx = tid + t * 256;
+            As[buf][idx >> 6][idx & 63] = ra[t];
+            Bs[buf][idx >> 4][idx & 15] = rb[t];
+        }
+    };
+    T acc = 0;
+    int buf = 0;
+    if (kbeg < kend) { load(kbeg); stash(0); }
+    __syncthreads();
+    for (int64_t k0 = kbeg; k0 < kend; k0 += BK) {
+        const bool more = k0 + BK < kend;
+        if (more) load(k0 + BK);
+#pragma unroll 16
+        for (int kk = 0; kk < BK; ++kk) acc += As[buf][ty][kk] * Bs[buf][kk][tx];
+        if (more) {
+            stash(buf ^ 1);
+            __syncthreads();
+            buf ^= 1;
+        }
+    }
+    const int64_t m = m0 + ty, n = n0 + tx;
+    if (m < ops.M && n < ops.N) {
+        if (partial == nullptr) ops.store(p, m, n, acc);
+        else {
+            T *dst = partial + ((int64_t)p * ops.M + m) * ops.N + n;
+            if (sizeof(T) == 8) atomicAdd((unsigned long long *)dst, (unsigned long long)acc);
+            else atomicAdd((unsigned int *)dst, (unsigned int)acc);
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------------------------
 // warp-per-row kernel for N <= NN (NN in {1, 2, 4, 8, 16})
 // ---------------------------------------------------------------------------------------------
 template <typename T>
@@ -348,8 +413,14 @@ psml_status launch_ring_gemm(const Ops &ops, T *ws, int64_t ws_words, cudaStream
     // split-K so the grid fills the GPU: ~2 CTAs (tiled) or ~16 warps (GEMV) per SM, each split
     // still >= 64 (tiled) / 256 (GEMV) deep.  Ring addition is exact, so partials are summed
     // with uint64/uint32 atomics and the epilogue runs once in ring_gemm_finalize.
+    const bool small = N > 16 && M * N * Ops::nparty <= ((int64_t)1 << 18);
     int splits = 1;
-    if (N <= 16) {
+    if (small) {
+        const int64_t tiles = ((M + 15) / 16) * ((N + 15) / 16) * Ops::nparty;
+        const int64_t target = (int64_t)sm_count * 2;
+        if (tiles < target && Kx > 512)
+            splits = (int)std::max<int64_t>(1, std::min<int64_t>((target + tiles - 1) / tiles, Kx / 256));
+    } else if (N <= 16) {
         const int64_t warps = M * Ops::nparty;
         const int64_t target = (int64_t)sm_count * 16;
         if (warps < target) splits = (int)std::max<int64_t>(1, std::min<int64_t>((target + warps - 1) / warps, Kx / 256));
@@ -366,7 +437,11 @@ psml_status launch_ring_gemm(const Ops &ops, T *ws, int64_t ws_words, cudaStream
     }
     int64_t kps = (Kx + splits - 1) / splits;
     ProfScope prof(PROF_GEMM, stream, (double)M * N * Kx * Ops::nparty);
-    if (N <= 16) {
+    if (small) {
+        kps = ((kps + 63) / 64) * 64;
+        dim3 grid((unsigned)((N + 15) / 16), (unsigned)((M + 15) / 16), (unsigned)(Ops::nparty * splits));
+        ring_gemm_small<T, Ops><<<grid, 256, 0, stream>>>(ops, kps, partial);
+    } else if (N <= 16) {
         const int64_t warps = M * Ops::nparty * splits;
         const int blocks = (int)((warps * 32 + 255) / 256);
         if (N == 1) ring_gemv<T, 1, Ops><<<blocks, 256, 0, stream>>>(ops, kps, splits, partial);

@@ -234,19 +234,6 @@ __global__ void hadamard_mask_kernel(CPair<T> A, CPair<T> B, CPair<T> U, CPair<T
     }
 }
 
-template <typename T>
-__global__ void hadamard_open_kernel(CPair<T> mE, CPair<T> mF, CPair<T> U, CPair<T> V, CPair<T> Z,
-                                     int64_t n, int trunc, Pair<T> C) {
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-        const T e = mE.p[0][i] + mE.p[1][i], f = mF.p[0][i] + mF.p[1][i];
-#pragma unroll
-        for (int p = 0; p < 2; ++p) {
-            T c = (T)p * e * f + e * V.p[p][i] + U.p[p][i] * f + Z.p[p][i];
-            C.p[p][i] = trunc_share<T>(c, p, trunc);
-        }
-    }
-}
-
 // ---------------------------------------------------------------------------------------------
 // Secure MSB chain (R9): Kogge-Stone carry on boolean shares, one kernel per round.
 // Input modes: 0 = x as given (n elements); 1 = Eq. 9 pair [z + h ; z - h] over z of n/2
@@ -278,20 +265,6 @@ __device__ __forceinline__ const T *mat_ptr(const MsbArgs<T> &a, int p, int t, i
     return a.mat.p[p] + ((int64_t)t * 3 + w) * a.n;
 }
 
-// Round 1: mask AND t = 0 with X = (x0, 0), Y = (0, x1).
-template <typename T>
-__global__ void msb_round0_kernel(MsbArgs<T> a) {
-    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < a.n; e += (int64_t)gridDim.x * blockDim.x) {
-#pragma unroll
-        for (int p = 0; p < 2; ++p) {
-            T x = msb_input(a, p, e);
-            T X = p == 0 ? x : (T)0, Y = p == 1 ? x : (T)0;
-            a.msg.p[p][e] = X ^ mat_ptr(a, p, 0, 0)[e];
-            a.msg.p[p][a.n + e] = Y ^ mat_ptr(a, p, 0, 1)[e];
-        }
-    }
-}
-
 // open one AND (message words w, w+1) of AND index t: returns both parties' z.
 template <typename T>
 __device__ __forceinline__ void and_open(const MsbArgs<T> &a, int64_t e, int w, int t, T z[2]) {
@@ -304,97 +277,189 @@ __device__ __forceinline__ void and_open(const MsbArgs<T> &a, int64_t e, int w, 
     }
 }
 
+// ---- per-element round bodies (one protocol round each) -----------------------------------------
+// Round 1: mask AND t = 0 with X = (x0, 0), Y = (0, x1).
+template <typename T>
+__device__ __forceinline__ void msb_round0_body(const MsbArgs<T> &a, int64_t e) {
+#pragma unroll
+    for (int p = 0; p < 2; ++p) {
+        T x = msb_input(a, p, e);
+        T X = p == 0 ? x : (T)0, Y = p == 1 ? x : (T)0;
+        a.msg.p[p][e] = X ^ mat_ptr(a, p, 0, 0)[e];
+        a.msg.p[p][a.n + e] = Y ^ mat_ptr(a, p, 0, 1)[e];
+    }
+}
+
 // Round j+1 (j = 1..L): open level j-1's ANDs, update G/P, mask level j's ANDs.
 template <typename T>
-__global__ void msb_level_kernel(MsbArgs<T> a, int j) {
+__device__ __forceinline__ void msb_level_body(const MsbArgs<T> &a, int j, int64_t e) {
     const int k = 1 << (j - 1);
-    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < a.n; e += (int64_t)gridDim.x * blockDim.x) {
-        T G[2], P[2], z[2];
-        if (j == 1) {
-            and_open(a, e, 0, 0, z);
+    T G[2], P[2], z[2];
+    if (j == 1) {
+        and_open(a, e, 0, 0, z);
 #pragma unroll
-            for (int p = 0; p < 2; ++p) { G[p] = z[p]; P[p] = msb_input(a, p, e); }
-        } else {
-            and_open(a, e, 0, 2 * j - 3, z);
-            T zp[2];
-            and_open(a, e, 2, 2 * j - 2, zp);
+        for (int p = 0; p < 2; ++p) { G[p] = z[p]; P[p] = msb_input(a, p, e); }
+    } else {
+        and_open(a, e, 0, 2 * j - 3, z);
+        T zp[2];
+        and_open(a, e, 2, 2 * j - 2, zp);
 #pragma unroll
-            for (int p = 0; p < 2; ++p) { G[p] = a.G.p[p][e] ^ z[p]; P[p] = zp[p]; }
+        for (int p = 0; p < 2; ++p) { G[p] = a.G.p[p][e] ^ z[p]; P[p] = zp[p]; }
+    }
+#pragma unroll
+    for (int p = 0; p < 2; ++p) {
+        const int t1 = 2 * j - 1;
+        a.msg.p[p][e] = P[p] ^ mat_ptr(a, p, t1, 0)[e];
+        a.msg.p[p][a.n + e] = (T)(G[p] << k) ^ mat_ptr(a, p, t1, 1)[e];
+        if (j < a.L) {
+            const int t2 = 2 * j;
+            a.msg.p[p][2 * a.n + e] = P[p] ^ mat_ptr(a, p, t2, 0)[e];
+            a.msg.p[p][3 * a.n + e] = (T)(P[p] << k) ^ mat_ptr(a, p, t2, 1)[e];
         }
-#pragma unroll
-        for (int p = 0; p < 2; ++p) {
-            const int t1 = 2 * j - 1;
-            a.msg.p[p][e] = P[p] ^ mat_ptr(a, p, t1, 0)[e];
-            a.msg.p[p][a.n + e] = (T)(G[p] << k) ^ mat_ptr(a, p, t1, 1)[e];
-            if (j < a.L) {
-                const int t2 = 2 * j;
-                a.msg.p[p][2 * a.n + e] = P[p] ^ mat_ptr(a, p, t2, 0)[e];
-                a.msg.p[p][3 * a.n + e] = (T)(P[p] << k) ^ mat_ptr(a, p, t2, 1)[e];
-            }
-            a.G.p[p][e] = G[p];
-            a.P.p[p][e] = P[p];
-        }
+        a.G.p[p][e] = G[p];
+        a.P.p[p][e] = P[p];
     }
 }
 
 // Round L+2: open the last G AND, msb_i = x_i[l-1] ^ G_i[l-2]; emit the B2A message c_i.
 template <typename T>
-__global__ void msb_final_kernel(MsbArgs<T> a, Pair<T> msbB) {
+__device__ __forceinline__ void msb_final_body(const MsbArgs<T> &a, const Pair<T> &msbB, int64_t e) {
     const int t = 2 * a.L - 1;
     const int64_t off = (int64_t)2 * a.L * 3 * a.n;
-    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < a.n; e += (int64_t)gridDim.x * blockDim.x) {
-        T z[2];
-        and_open(a, e, 0, t, z);
+    T z[2];
+    and_open(a, e, 0, t, z);
 #pragma unroll
-        for (int p = 0; p < 2; ++p) {
-            T G = a.G.p[p][e] ^ z[p];
-            T x = msb_input(a, p, e);
-            T b = ((x >> (a.l - 1)) & 1) ^ ((G >> (a.l - 2)) & 1);
-            if (msbB.p[p]) msbB.p[p][e] = b;
-            a.msg.p[p][e] = b ^ a.mat.p[p][off + e];   // c_i = msb_i ^ rB_i
-        }
+    for (int p = 0; p < 2; ++p) {
+        T G = a.G.p[p][e] ^ z[p];
+        T x = msb_input(a, p, e);
+        T b = ((x >> (a.l - 1)) & 1) ^ ((G >> (a.l - 2)) & 1);
+        if (msbB.p[p]) msbB.p[p][e] = b;
+        a.msg.p[p][e] = b ^ a.mat.p[p][off + e];   // c_i = msb_i ^ rB_i
     }
 }
 
 // Round L+3: open c, [msb]^A; then either store msbA (what = 0) or, for ReLU/Eq. 9 (what = 1),
 // form drelu_i = [i==0] - msbA_i and mask the Hadamard x . drelu (messages mE, mF).
 template <typename T>
-__global__ void msb_b2a_kernel(MsbArgs<T> a, Pair<T> msbA, Pair<T> drelu, CPair<T> U, CPair<T> V,
-                               Pair<T> mE, Pair<T> mF, int what) {
+__device__ __forceinline__ void msb_b2a_body(const MsbArgs<T> &a, const Pair<T> &msbA, const Pair<T> &drelu,
+                                             const CPair<T> &U, const CPair<T> &V, const Pair<T> &mE,
+                                             const Pair<T> &mF, int what, int64_t e) {
     const int64_t off = (int64_t)2 * a.L * 3 * a.n;
-    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < a.n; e += (int64_t)gridDim.x * blockDim.x) {
-        const T c = a.msg.p[0][e] ^ a.msg.p[1][e];
-        const T s = (T)1 - (T)2 * c;
+    const T c = a.msg.p[0][e] ^ a.msg.p[1][e];
+    const T s = (T)1 - (T)2 * c;
 #pragma unroll
-        for (int p = 0; p < 2; ++p) {
-            T m = (p == 0 ? c : (T)0) + s * a.mat.p[p][off + a.n + e];
-            if (what == 0) {
-                msbA.p[p][e] = m;
-            } else {
-                T d = (p == 0 ? (T)1 : (T)0) - m;
-                if (drelu.p[p]) drelu.p[p][e] = d;
-                mE.p[p][e] = msb_input(a, p, e) - U.p[p][e];
-                mF.p[p][e] = d - V.p[p][e];
-            }
+    for (int p = 0; p < 2; ++p) {
+        T m = (p == 0 ? c : (T)0) + s * a.mat.p[p][off + a.n + e];
+        if (what == 0) {
+            msbA.p[p][e] = m;
+        } else {
+            T d = (p == 0 ? (T)1 : (T)0) - m;
+            if (drelu.p[p]) drelu.p[p][e] = d;
+            mE.p[p][e] = msb_input(a, p, e) - U.p[p][e];
+            mF.p[p][e] = d - V.p[p][e];
         }
+    }
+}
+
+template <typename T>
+__device__ __forceinline__ void hadamard_open_body(const CPair<T> &mE, const CPair<T> &mF, const CPair<T> &U,
+                                                   const CPair<T> &V, const CPair<T> &Z, int trunc,
+                                                   const Pair<T> &C, int64_t i) {
+    const T e = mE.p[0][i] + mE.p[1][i], f = mF.p[0][i] + mF.p[1][i];
+#pragma unroll
+    for (int p = 0; p < 2; ++p) {
+        T c = (T)p * e * f + e * V.p[p][i] + U.p[p][i] * f + Z.p[p][i];
+        C.p[p][i] = trunc_share<T>(c, p, trunc);
     }
 }
 
 // Round L+4 for Eq. 9: open the Hadamard of 2n' elements, y_i = r_i[e] - r_i[e + n'].
 template <typename T>
+__device__ __forceinline__ void eq9_open_body(const CPair<T> &mE, const CPair<T> &mF, const CPair<T> &U,
+                                              const CPair<T> &V, const CPair<T> &Z, int64_t nh, const Pair<T> &y,
+                                              const CPair<T> &Ysub, const Pair<T> &delta, int64_t e) {
+    const T e1 = mE.p[0][e] + mE.p[1][e], f1 = mF.p[0][e] + mF.p[1][e];
+    const T e2 = mE.p[0][e + nh] + mE.p[1][e + nh], f2 = mF.p[0][e + nh] + mF.p[1][e + nh];
+#pragma unroll
+    for (int p = 0; p < 2; ++p) {
+        T r1 = (T)p * e1 * f1 + e1 * V.p[p][e] + U.p[p][e] * f1 + Z.p[p][e];
+        T r2 = (T)p * e2 * f2 + e2 * V.p[p][e + nh] + U.p[p][e + nh] * f2 + Z.p[p][e + nh];
+        T out = r1 - r2;
+        if (y.p[p]) y.p[p][e] = out;
+        if (delta.p[p]) delta.p[p][e] = out - Ysub.p[p][e];
+    }
+}
+
+#define PSML_GRID_LOOP(e, n) \
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < (n); e += (int64_t)gridDim.x * blockDim.x)
+
+// ---- one kernel per round (the split-deployment structure; also the fallback) --------------------
+template <typename T>
+__global__ void msb_round0_kernel(MsbArgs<T> a) { PSML_GRID_LOOP(e, a.n) msb_round0_body(a, e); }
+
+template <typename T>
+__global__ void msb_level_kernel(MsbArgs<T> a, int j) { PSML_GRID_LOOP(e, a.n) msb_level_body(a, j, e); }
+
+template <typename T>
+__global__ void msb_final_kernel(MsbArgs<T> a, Pair<T> msbB) { PSML_GRID_LOOP(e, a.n) msb_final_body(a, msbB, e); }
+
+template <typename T>
+__global__ void msb_b2a_kernel(MsbArgs<T> a, Pair<T> msbA, Pair<T> drelu, CPair<T> U, CPair<T> V,
+                               Pair<T> mE, Pair<T> mF, int what) {
+    PSML_GRID_LOOP(e, a.n) msb_b2a_body(a, msbA, drelu, U, V, mE, mF, what, e);
+}
+
+template <typename T>
+__global__ void hadamard_open_kernel(CPair<T> mE, CPair<T> mF, CPair<T> U, CPair<T> V, CPair<T> Z,
+                                     int64_t n, int trunc, Pair<T> C) {
+    PSML_GRID_LOOP(i, n) hadamard_open_body(mE, mF, U, V, Z, trunc, C, i);
+}
+
+template <typename T>
 __global__ void eq9_open_kernel(CPair<T> mE, CPair<T> mF, CPair<T> U, CPair<T> V, CPair<T> Z,
                                 int64_t nh, Pair<T> y, CPair<T> Ysub, Pair<T> delta) {
-    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < nh; e += (int64_t)gridDim.x * blockDim.x) {
-        const T e1 = mE.p[0][e] + mE.p[1][e], f1 = mF.p[0][e] + mF.p[1][e];
-        const T e2 = mE.p[0][e + nh] + mE.p[1][e + nh], f2 = mF.p[0][e + nh] + mF.p[1][e + nh];
-#pragma unroll
-        for (int p = 0; p < 2; ++p) {
-            T r1 = (T)p * e1 * f1 + e1 * V.p[p][e] + U.p[p][e] * f1 + Z.p[p][e];
-            T r2 = (T)p * e2 * f2 + e2 * V.p[p][e + nh] + U.p[p][e + nh] * f2 + Z.p[p][e + nh];
-            T out = r1 - r2;
-            if (y.p[p]) y.p[p][e] = out;
-            if (delta.p[p]) delta.p[p][e] = out - Ysub.p[p][e];
+    PSML_GRID_LOOP(e, nh) eq9_open_body(mE, mF, U, V, Z, nh, y, Ysub, delta, e);
+}
+
+// ---- the whole chain in ONE launch, rounds in order per element ----------------------------------
+// In the co-resident engine, round r+1 of element e only opens the two parties' round-r messages
+// of the same element e.  One thread therefore runs element e through every round in protocol
+// order -- each round still writes both parties' masked messages to their send buffers and the
+// next round opens them from there -- so the chain costs one launch instead of one per round.
+// (A split deployment exchanges the messages between rounds instead: msb_*_kernel per round.)
+// Eq. 9 pairs element e with e + n/2 so its final opening stays thread-local.
+template <typename T>
+struct ChainOut {
+    Pair<T> msbA, msbB, drelu, y, delta;
+    CPair<T> U, V, Z, Ysub;
+    Pair<T> mE, mF;
+    int what;
+};
+
+template <typename T>
+__device__ __forceinline__ void msb_chain_element(const MsbArgs<T> &a, const ChainOut<T> &o, int64_t e) {
+    msb_round0_body(a, e);
+#pragma unroll 1
+    for (int j = 1; j <= a.L; ++j) msb_level_body(a, j, e);
+    msb_final_body(a, o.msbB, e);
+    msb_b2a_body(a, o.msbA, o.drelu, o.U, o.V, o.mE, o.mF, o.what == 0 ? 0 : 1, e);
+}
+
+template <typename T>
+__global__ void __launch_bounds__(256) msb_chain_fused_kernel(MsbArgs<T> a, ChainOut<T> o) {
+    CPair<T> ce{{o.mE.p[0], o.mE.p[1]}}, cf{{o.mF.p[0], o.mF.p[1]}};
+    if (o.what == 2) {
+        const int64_t nh = a.n / 2;
+        PSML_GRID_LOOP(e, nh) {
+            msb_chain_element(a, o, e);
+            msb_chain_element(a, o, e + nh);
+            eq9_open_body(ce, cf, o.U, o.V, o.Z, nh, o.y, o.Ysub, o.delta, e);
         }
+        return;
+    }
+    PSML_GRID_LOOP(e, a.n) {
+        msb_chain_element(a, o, e);
+        if (o.what == 1) hadamard_open_body(ce, cf, o.U, o.V, o.Z, 0, o.y, e);
     }
 }
 

@@ -3,6 +3,7 @@
 // model step allocates nothing (and can be captured in a CUDA graph).
 #pragma once
 #include <algorithm>
+#include <cstdlib>
 
 #include "common.cuh"
 #include "gemm_simt.cuh"
@@ -11,6 +12,17 @@
 namespace psml {
 
 constexpr int EW_THREADS = 256;
+
+// MSB chain execution: 0 = one launch running each element through every round in order,
+// 1 = one kernel per round.  Environment override PSML_MSB_CHAIN=rounds (tests compare both).
+inline int chain_mode() {
+    static int m = -1;
+    if (m < 0) {
+        const char *e = getenv("PSML_MSB_CHAIN");
+        m = (e && e[0] == 'r') ? 1 : 0;
+    }
+    return m;
+}
 
 inline int ew_grid(int64_t n) { return grid_for(n, EW_THREADS, 148 * 32); }
 
@@ -152,35 +164,47 @@ psml_status msb_chain(const T *const x[2], int64_t n, const T *const mat[2], int
     a.P = Pair<T>{{ws + 2 * n, ws + 3 * n}};
     a.msg = Pair<T>{{ws + 4 * n, ws + 8 * n}};
     a.n = n; a.mode = mode; a.half = half; a.L = ilog2_int(l); a.l = l;
-    const int g = ew_grid(n);
     // algorithmic bytes of the chain (both parties): per AND round each party reads 2 message
     // words of both parties + 3 material words + state and writes state + 2 messages
     ProfScope prof(PROF_MSB, s, (double)sizeof(T) * n * (2.0 * (a.L + 2) * 14 + 16));
+    Pair<T> mE{{a.msg.p[0] + n, a.msg.p[1] + n}}, mF{{a.msg.p[0] + 2 * n, a.msg.p[1] + 2 * n}};
+    ChainOut<T> o;
+    o.msbA = Pair<T>{{msbA ? msbA[0] : nullptr, msbA ? msbA[1] : nullptr}};
+    o.msbB = Pair<T>{{msbB ? msbB[0] : nullptr, msbB ? msbB[1] : nullptr}};
+    o.drelu = Pair<T>{{drelu ? drelu[0] : nullptr, drelu ? drelu[1] : nullptr}};
+    o.y = Pair<T>{{y ? y[0] : nullptr, y ? y[1] : nullptr}};
+    o.delta = Pair<T>{{delta ? delta[0] : nullptr, delta ? delta[1] : nullptr}};
+    o.U = CPair<T>{{U ? U[0] : nullptr, U ? U[1] : nullptr}};
+    o.V = CPair<T>{{V ? V[0] : nullptr, V ? V[1] : nullptr}};
+    o.Z = CPair<T>{{Z ? Z[0] : nullptr, Z ? Z[1] : nullptr}};
+    o.Ysub = CPair<T>{{Ysub ? Ysub[0] : nullptr, Ysub ? Ysub[1] : nullptr}};
+    o.mE = mE;
+    o.mF = mF;
+    o.what = what;
+    if (chain_mode() == 0) {   // all rounds of an element in one thread, one launch
+        const int64_t units = what == 2 ? n / 2 : n;
+        msb_chain_fused_kernel<T><<<ew_grid(units), EW_THREADS, 0, s>>>(a, o);
+        PSML_LAUNCH_CHECK();
+        return PSML_OK;
+    }
+    const int g = ew_grid(n);
     msb_round0_kernel<T><<<g, EW_THREADS, 0, s>>>(a);
     PSML_LAUNCH_CHECK();
     for (int j = 1; j <= a.L; ++j) {
         msb_level_kernel<T><<<g, EW_THREADS, 0, s>>>(a, j);
         PSML_LAUNCH_CHECK();
     }
-    Pair<T> mb{{msbB ? msbB[0] : nullptr, msbB ? msbB[1] : nullptr}};
-    msb_final_kernel<T><<<g, EW_THREADS, 0, s>>>(a, mb);
+    msb_final_kernel<T><<<g, EW_THREADS, 0, s>>>(a, o.msbB);
     PSML_LAUNCH_CHECK();
-    Pair<T> mE{{a.msg.p[0] + n, a.msg.p[1] + n}}, mF{{a.msg.p[0] + 2 * n, a.msg.p[1] + 2 * n}};
-    Pair<T> ma{{msbA ? msbA[0] : nullptr, msbA ? msbA[1] : nullptr}};
-    Pair<T> dr{{drelu ? drelu[0] : nullptr, drelu ? drelu[1] : nullptr}};
-    CPair<T> u{{U ? U[0] : nullptr, U ? U[1] : nullptr}}, v{{V ? V[0] : nullptr, V ? V[1] : nullptr}};
-    msb_b2a_kernel<T><<<g, EW_THREADS, 0, s>>>(a, ma, dr, u, v, mE, mF, what == 0 ? 0 : 1);
+    msb_b2a_kernel<T><<<g, EW_THREADS, 0, s>>>(a, o.msbA, o.drelu, o.U, o.V, mE, mF, what == 0 ? 0 : 1);
     PSML_LAUNCH_CHECK();
     if (what == 0) return PSML_OK;
-    CPair<T> ce{{mE.p[0], mE.p[1]}}, cf{{mF.p[0], mF.p[1]}}, z{{Z[0], Z[1]}};
+    CPair<T> ce{{mE.p[0], mE.p[1]}}, cf{{mF.p[0], mF.p[1]}};
     if (what == 1) {
-        hadamard_open_kernel<T><<<g, EW_THREADS, 0, s>>>(ce, cf, u, v, z, n, 0, Pair<T>{{y[0], y[1]}});
+        hadamard_open_kernel<T><<<g, EW_THREADS, 0, s>>>(ce, cf, o.U, o.V, o.Z, n, 0, o.y);
     } else {
         const int64_t nh = n / 2;
-        Pair<T> yy{{y ? y[0] : nullptr, y ? y[1] : nullptr}};
-        CPair<T> ys{{Ysub ? Ysub[0] : nullptr, Ysub ? Ysub[1] : nullptr}};
-        Pair<T> dd{{delta ? delta[0] : nullptr, delta ? delta[1] : nullptr}};
-        eq9_open_kernel<T><<<ew_grid(nh), EW_THREADS, 0, s>>>(ce, cf, u, v, z, nh, yy, ys, dd);
+        eq9_open_kernel<T><<<ew_grid(nh), EW_THREADS, 0, s>>>(ce, cf, o.U, o.V, o.Z, nh, o.y, o.Ysub, o.delta);
     }
     PSML_LAUNCH_CHECK();
     return PSML_OK;

@@ -258,3 +258,15 @@ def test_delta_codec(P, orc, ctx, frac_changed):
     t = to_dev(prev, l)
     P.delta_apply(ctx, t, got)
     assert np.array_equal(to_np(t), cur)
+
+
+def test_msb_chain_per_round_kernels_match():
+    """The one-kernel-per-round chain (split-deployment structure) gives the same shares as the
+    cooperative single-launch chain: rerun the activation parity tests with PSML_MSB_CHAIN=rounds."""
+    import subprocess
+    import sys
+    env = dict(os.environ, PSML_MSB_CHAIN="rounds")
+    r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu", "-k",
+                        "test_secure_msb_relu_eq9", __file__], env=env, capture_output=True, text=True,
+                       cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
