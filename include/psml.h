@@ -160,6 +160,23 @@ psml_status psml_secure_matmul(psml_ctx ctx, const void *const A[2], const void 
                                const void *const Z[2], int64_t M, int64_t K, int64_t N,
                                int32_t flags, int32_t trunc_bits, void *const C[2],
                                const psml_trace *trace, psml_stream stream);
+/* Split deployment: ONE party per process / GPU (Fig. 1b: two servers).  The Beaver
+ * product becomes two calls around the caller's exchange of the masked messages:
+ *  round 1  psml_beaver_mask: E_send = op(A)_i - U_i (M x K), F_send = op(B)_i - V_i (K x N)
+ *           (Eq. 4); the caller sends E_send, F_send to the peer and receives the peer's
+ *           E_recv, F_recv (e.g. NCCL send/recv over NVLink; uint64/uint32 words).
+ *  round 2  psml_beaver_open_matmul: E = E_send + E_recv, F = F_send + F_recv (Eq. 5) opened
+ *           inside the GEMM's operand loads, C_i = i.E.F + E.V_i + U_i.F + Z_i (Eq. 8 shape),
+ *           then truncation by trunc_bits.  Bit-identical to psml_secure_matmul's party-i share.
+ * Buffers are caller-owned device memory; the two calls must use the same shapes and flags. */
+psml_status psml_beaver_mask(psml_ctx ctx, int32_t party, const void *A_i, const void *B_i,
+                             const void *U_i, const void *V_i, int64_t M, int64_t K, int64_t N,
+                             int32_t flags, void *E_send, void *F_send, psml_stream stream);
+psml_status psml_beaver_open_matmul(psml_ctx ctx, int32_t party, const void *E_send,
+                                    const void *E_recv, const void *F_send, const void *F_recv,
+                                    const void *U_i, const void *V_i, const void *Z_i, int64_t M,
+                                    int64_t K, int64_t N, int32_t trunc_bits, void *C_i,
+                                    psml_stream stream);
 /* Beaver Hadamard product of n elements: C_i = i.E.F + E.V_i + U_i.F + Z_i elementwise. */
 psml_status psml_secure_hadamard(psml_ctx ctx, const void *const A[2], const void *const B[2],
                                  const void *const U[2], const void *const V[2],

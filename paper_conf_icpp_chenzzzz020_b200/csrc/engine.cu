@@ -349,6 +349,68 @@ psml_status psml_secure_matmul(psml_ctx ctx, const void *const A[2], const void 
     return secure_matmul_t<uint32_t>(c, A, B, U, V, Z, M, K, N, flags, trunc_bits, C, trace, s);
 }
 
+template <typename T>
+static psml_status beaver_mask_t(const void *A, const void *B, const void *U, const void *V, int64_t M, int64_t K,
+                                 int64_t N, int32_t flags, void *E, void *F, cudaStream_t s) {
+    MaskJobs<T> jobs;
+    jobs.j[0] = {(const T *)A, (const T *)U, (T *)E, M, K, (flags & PSML_TRANS_A) ? 1 : 0};
+    jobs.j[1] = {(const T *)B, (const T *)V, (T *)F, K, N, (flags & PSML_TRANS_B) ? 1 : 0};
+    jobs.count = 2;
+    const int64_t maxt = std::max(((M + 31) / 32) * ((K + 31) / 32), ((K + 31) / 32) * ((N + 31) / 32));
+    ProfScope prof(PROF_MASK, s, 3.0 * sizeof(T) * (M * K + K * N));
+    mask_kernel<T><<<dim3((unsigned)std::min<int64_t>(maxt, 148 * 8), 1, 2), dim3(32, 8), 0, s>>>(jobs);
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
+psml_status psml_beaver_mask(psml_ctx ctx, int32_t party, const void *A_i, const void *B_i, const void *U_i,
+                             const void *V_i, int64_t M, int64_t K, int64_t N, int32_t flags, void *E_send,
+                             void *F_send, psml_stream stream) {
+    if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
+    Ctx *c = reinterpret_cast<Ctx *>(ctx);
+    if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
+    if (M <= 0 || K <= 0 || N <= 0) return fail(PSML_ERR_SHAPE, "M, K, N must be positive");
+    if (flags & ~(PSML_TRANS_A | PSML_TRANS_B)) return fail(PSML_ERR_INVALID, "flags: TRANS_A / TRANS_B only");
+    PSML_TRY(check_ptrs({A_i, B_i, U_i, V_i, E_send, F_send}));
+    cudaStream_t s = (cudaStream_t)stream;
+    if (c->ring.l == 64) return beaver_mask_t<uint64_t>(A_i, B_i, U_i, V_i, M, K, N, flags, E_send, F_send, s);
+    return beaver_mask_t<uint32_t>(A_i, B_i, U_i, V_i, M, K, N, flags, E_send, F_send, s);
+}
+
+template <typename T>
+static psml_status open_matmul_t(Ctx *c, int party, const void *Es, const void *Er, const void *Fs, const void *Fr,
+                                 const void *U, const void *V, const void *Z, int64_t M, int64_t K, int64_t N,
+                                 int trunc, void *C, cudaStream_t s) {
+    if (c->use_tc(M, 2 * K, N)) {
+        psml_status st = tc_open_matmul_one(c, 8 * (int)sizeof(T), party, Es, Er, Fs, Fr, U, V, Z, M, K, N, trunc, C, s);
+        if (st != PSML_ERR_UNSUPPORTED) return st;
+    }
+    PSML_TRY(c->ensure_ws(sizeof(T) * M * N));
+    BeaverOps1<T> ops;
+    ops.mE0 = (const T *)Es; ops.mE1 = (const T *)Er; ops.mF0 = (const T *)Fs; ops.mF1 = (const T *)Fr;
+    ops.U = (const T *)U; ops.V = (const T *)V; ops.Z = (const T *)Z; ops.C = (T *)C;
+    ops.M = M; ops.N = N; ops.K = K; ops.Kext = 2 * K; ops.party = party; ops.trunc = trunc;
+    return launch_ring_gemm<T, BeaverOps1<T>>(ops, (T *)c->ws, M * N, s, c->sm_count);
+}
+
+psml_status psml_beaver_open_matmul(psml_ctx ctx, int32_t party, const void *E_send, const void *E_recv,
+                                    const void *F_send, const void *F_recv, const void *U_i, const void *V_i,
+                                    const void *Z_i, int64_t M, int64_t K, int64_t N, int32_t trunc_bits, void *C_i,
+                                    psml_stream stream) {
+    if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
+    Ctx *c = reinterpret_cast<Ctx *>(ctx);
+    if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
+    if (M <= 0 || K <= 0 || N <= 0) return fail(PSML_ERR_SHAPE, "M, K, N must be positive");
+    if (trunc_bits < 0 || trunc_bits >= c->ring.l) return fail(PSML_ERR_SHAPE, "trunc_bits must be in [0, l)");
+    PSML_TRY(check_ptrs({E_send, E_recv, F_send, F_recv, U_i, V_i, Z_i, C_i}));
+    cudaStream_t s = (cudaStream_t)stream;
+    if (c->ring.l == 64)
+        return open_matmul_t<uint64_t>(c, party, E_send, E_recv, F_send, F_recv, U_i, V_i, Z_i, M, K, N, trunc_bits,
+                                       C_i, s);
+    return open_matmul_t<uint32_t>(c, party, E_send, E_recv, F_send, F_recv, U_i, V_i, Z_i, M, K, N, trunc_bits, C_i,
+                                   s);
+}
+
 psml_status psml_secure_hadamard(psml_ctx ctx, const void *const A[2], const void *const B[2], const void *const U[2],
                                  const void *const V[2], const void *const Z[2], int64_t n, int32_t trunc_bits,
                                  void *const C[2], psml_stream stream) {

@@ -19,11 +19,13 @@ struct Ctx {
     void *ws = nullptr;
     size_t ws_bytes = 0;
     psml_status ensure_ws(size_t bytes);
-    // tcgen05 limb GEMM pays once the product has enough tiles and depth (gemm_tc.cu).
+    // tcgen05 limb GEMM pays once a party's product has >= 2^25 ring MACs (measured on B200:
+    // 128x1568x128 is 2x faster on CUDA cores, 12544x256x64 1.5x and 1024^3 10x faster on tcgen05;
+    // tools/mm_prof.py).
     bool use_tc(int64_t M, int64_t Kext, int64_t N) const {
         if (!tc_ok || backend == 1) return false;
         if (backend == 2) return true;
-        return M >= 256 && N >= 128 && Kext >= 256 && M * N >= (int64_t)1 << 18;
+        return M >= 128 && N >= 64 && M * N * Kext >= ((int64_t)1 << 25);
     }
 };
 
@@ -70,6 +72,18 @@ psml_status trace_opened(Ctx *c, int64_t M, int64_t K, int64_t N, const psml_tra
 
 psml_status tc_dealer_gemm(int l, const void *U0, const void *U1, const void *V0, const void *V1, int64_t M, int64_t K,
                            int64_t N, const void *Z0, void *Z1, void *ws, size_t ws_bytes, cudaStream_t s);
+
+template <typename T>
+size_t tc_beaver_ws_bytes(int64_t M, int64_t K, int64_t N);
+template <typename T>
+psml_status tc_beaver_matmul_ws(const T *const A[2], const T *const B[2], const T *const U[2], const T *const V[2],
+                                const T *const Z[2], int64_t M, int64_t K, int64_t N, int flags, int trunc,
+                                T *const C[2], void *ws, size_t ws_bytes, int sm_count, cudaStream_t s);
+
+// Split-deployment round 2 on tcgen05 for one party (gemm_tc.cu).
+psml_status tc_open_matmul_one(Ctx *c, int l, int party, const void *Es, const void *Er, const void *Fs,
+                               const void *Fr, const void *U, const void *V, const void *Z, int64_t M, int64_t K,
+                               int64_t N, int trunc, void *C, cudaStream_t s);
 
 // tcgen05 Beaver product (gemm_tc.cu); PSML_ERR_UNSUPPORTED = take the CUDA-core path.
 template <typename T>

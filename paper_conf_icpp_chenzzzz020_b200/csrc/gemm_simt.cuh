@@ -89,13 +89,50 @@ struct BeaverOps {
     }
 };
 
+// One party of the split deployment: own messages (mE0/mF0 = sent) + the peer's (mE1/mF1 =
+// received); same arithmetic as BeaverOps for party `party`.
+template <typename T>
+struct BeaverOps1 {
+    const T *mE0, *mE1, *mF0, *mF1;
+    const T *U, *V, *Z;
+    T *C;
+    int64_t M, N, K, Kext;
+    int party, trunc;
+    static constexpr int nparty = 1;
+    __device__ __forceinline__ T a(int, int64_t m, int64_t k) const {
+        if (k < K) {
+            const T e = mE0[m * K + k] + mE1[m * K + k];
+            return (T)((T)party * e + U[m * K + k]);
+        }
+        k -= K;
+        return mE0[m * K + k] + mE1[m * K + k];
+    }
+    __device__ __forceinline__ T b(int, int64_t k, int64_t n) const {
+        if (k < K) return mF0[k * N + n] + mF1[k * N + n];
+        return V[(k - K) * N + n];
+    }
+    __device__ __forceinline__ void store(int, int64_t m, int64_t n, T acc) const {
+        C[m * N + n] = trunc_share<T>(acc + Z[m * N + n], party, trunc);
+    }
+};
+
 // Convolution as im2col ring GEMM with the mask applied to the UN-EXPANDED input (R17):
 // E_X = E_0 + E_1 over B x (C H W); im2col row r = (b, oy, ox), col c = (ch, ky, kx).
 // transposed = 0: A' = im2col(.)            (rows B*OH*OW, K = C*k*k)   -- conv forward
 // transposed = 1: A' = im2col(.)^T          (rows C*k*k,  K = B*OH*OW)  -- weight gradient
 struct ConvGeom {
     int C, H, W, k, OH, OW;
+    const int32_t *coloff;   // device table: offset of im2col column c = (ch, ky, kx) in a sample
 };
+
+// im2col source index of (row r = (b, oy, ox), column c): 32-bit row decomposition (indices of
+// the paper's workloads fit in 31 bits) + the precomputed column offset -- no 64-bit divisions.
+__device__ __forceinline__ int64_t conv_src(const ConvGeom &g, int64_t r, int64_t c) {
+    const uint32_t r32 = (uint32_t)r, plane = (uint32_t)(g.OH * g.OW);
+    const uint32_t b = r32 / plane, rem = r32 - b * plane;
+    const uint32_t oy = rem / (uint32_t)g.OW, ox = rem - oy * (uint32_t)g.OW;
+    return (int64_t)b * ((int64_t)g.C * g.H * g.W) + (int64_t)(oy * (uint32_t)g.W + ox) + g.coloff[c];
+}
 
 template <typename T>
 struct ConvBeaverOps {
@@ -108,15 +145,7 @@ struct ConvBeaverOps {
     int64_t M, N, K, Kext;
     int transposed, trunc;
     static constexpr int nparty = 2;
-    __device__ __forceinline__ int64_t src(int64_t r, int64_t c) const {
-        int64_t plane = (int64_t)g.OH * g.OW;
-        int64_t b = r / plane, rem = r - b * plane;
-        int oy = (int)(rem / g.OW), ox = (int)(rem - (int64_t)oy * g.OW);
-        int kk = g.k * g.k;
-        int ch = (int)(c / kk), r2 = (int)(c - (int64_t)ch * kk);
-        int ky = r2 / g.k, kx = r2 - ky * g.k;
-        return b * ((int64_t)g.C * g.H * g.W) + ((int64_t)ch * g.H + oy + ky) * g.W + ox + kx;
-    }
+    __device__ __forceinline__ int64_t src(int64_t r, int64_t c) const { return conv_src(g, r, c); }
     __device__ __forceinline__ T a(int p, int64_t m, int64_t k) const {
         bool first = k < K;
         if (!first) k -= K;
@@ -145,15 +174,7 @@ struct ConvDealerOps {
     int64_t M, N, Kext;
     int transposed;
     static constexpr int nparty = 1;
-    __device__ __forceinline__ int64_t src(int64_t r, int64_t c) const {
-        int64_t plane = (int64_t)g.OH * g.OW;
-        int64_t b = r / plane, rem = r - b * plane;
-        int oy = (int)(rem / g.OW), ox = (int)(rem - (int64_t)oy * g.OW);
-        int kk = g.k * g.k;
-        int ch = (int)(c / kk), r2 = (int)(c - (int64_t)ch * kk);
-        int ky = r2 / g.k, kx = r2 - ky * g.k;
-        return b * ((int64_t)g.C * g.H * g.W) + ((int64_t)ch * g.H + oy + ky) * g.W + ox + kx;
-    }
+    __device__ __forceinline__ int64_t src(int64_t r, int64_t c) const { return conv_src(g, r, c); }
     __device__ __forceinline__ T a(int, int64_t m, int64_t k) const {
         int64_t s = transposed ? src(k, m) : src(m, k);
         return U0[s] + U1[s];
@@ -413,14 +434,18 @@ psml_status launch_ring_gemm(const Ops &ops, T *ws, int64_t ws_words, cudaStream
     // split-K so the grid fills the GPU: ~2 CTAs (tiled) or ~16 warps (GEMV) per SM, each split
     // still >= 64 (tiled) / 256 (GEMV) deep.  Ring addition is exact, so partials are summed
     // with uint64/uint32 atomics and the epilogue runs once in ring_gemm_finalize.
-    const bool small = N > 16 && M * N * Ops::nparty <= ((int64_t)1 << 18);
+    // kernel choice: warp-per-row GEMV for skinny outputs with few rows (w^T x, MLP output layer),
+    // the 16 x 16 small-tile kernel for small outputs or skinny outputs with many rows (CNN conv
+    // im2col GEMMs), the 64 x 64 register-blocked kernel otherwise.
+    const bool gemv = N <= 16 && M * Ops::nparty <= 4096;
+    const bool small = !gemv && (N <= 16 || M * N * Ops::nparty <= ((int64_t)1 << 18));
     int splits = 1;
     if (small) {
         const int64_t tiles = ((M + 15) / 16) * ((N + 15) / 16) * Ops::nparty;
-        const int64_t target = (int64_t)sm_count * 2;
+        const int64_t target = (int64_t)sm_count * (Kx >= 16384 ? 4 : 2);
         if (tiles < target && Kx > 512)
             splits = (int)std::max<int64_t>(1, std::min<int64_t>((target + tiles - 1) / tiles, Kx / 256));
-    } else if (N <= 16) {
+    } else if (gemv) {
         const int64_t warps = M * Ops::nparty;
         const int64_t target = (int64_t)sm_count * 16;
         if (warps < target) splits = (int)std::max<int64_t>(1, std::min<int64_t>((target + warps - 1) / warps, Kx / 256));
@@ -441,7 +466,7 @@ psml_status launch_ring_gemm(const Ops &ops, T *ws, int64_t ws_words, cudaStream
         kps = ((kps + 63) / 64) * 64;
         dim3 grid((unsigned)((N + 15) / 16), (unsigned)((M + 15) / 16), (unsigned)(Ops::nparty * splits));
         ring_gemm_small<T, Ops><<<grid, 256, 0, stream>>>(ops, kps, partial);
-    } else if (N <= 16) {
+    } else if (gemv) {
         const int64_t warps = M * Ops::nparty * splits;
         const int blocks = (int)((warps * 32 + 255) / 256);
         if (N == 1) ring_gemv<T, 1, Ops><<<blocks, 256, 0, stream>>>(ops, kps, splits, partial);

@@ -186,6 +186,7 @@ struct TcParams {
     int kb_per_split;
     int64_t M, N;
     int nparty;
+    int party_base;    // party of blockIdx.z % nparty == 0 (split deployment: the local party)
     int mode;          // 0 plain store, 1 Beaver (+Z_i, trunc), 2 dealer (Z1 = acc - Z0), 3 atomic partial
     T *C[2];
     const T *Z[2];
@@ -213,7 +214,7 @@ __device__ __forceinline__ void epi_chunk(T *st, const T v[16], int lane, int64_
         const T x = st[rl * 17 + c];
         const int64_t o = row * P.N + col;
         if (P.mode == 3) {
-            T *dst = P.partial + (int64_t)party * P.M * P.N + o;
+            T *dst = P.partial + (int64_t)(party - P.party_base) * P.M * P.N + o;
             if (sizeof(T) == 8) atomicAdd((unsigned long long *)dst, (unsigned long long)x);
             else atomicAdd((unsigned int *)dst, (unsigned int)x);
             continue;
@@ -242,7 +243,7 @@ __global__ void __launch_bounds__(128, 1) tc_ring_gemm_kernel(const TcParams<T> 
     uint32_t *tmem_slot = (uint32_t *)(accum + 1);
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int party = blockIdx.z % P.nparty, split = blockIdx.z / P.nparty;
+    const int party = P.party_base + blockIdx.z % P.nparty, split = blockIdx.z / P.nparty;
     const int nb = blockIdx.x, rb = blockIdx.y;
     const int nkb = P.nkb_lo + P.nkb_hi;
     const int kb0 = split * P.kb_per_split;
@@ -361,7 +362,7 @@ __global__ void __launch_bounds__(192, 1) tc_ring_gemm64_v2(const TcParams<uint6
     uint32_t *tmem_slot = (uint32_t *)(acce + 1);
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int party = blockIdx.z % P.nparty, split = blockIdx.z / P.nparty;
+    const int party = P.party_base + blockIdx.z % P.nparty, split = blockIdx.z / P.nparty;
     const int nb = blockIdx.x, rb = blockIdx.y;
     const int nkb = P.nkb_lo + P.nkb_hi;
     const int kb0 = split * P.kb_per_split;
@@ -481,7 +482,7 @@ __global__ void __launch_bounds__(192, 1) tc_ring_gemm64_v2(const TcParams<uint6
                     const int64_t col = col0 + j0 + j;
                     if (col >= P.N) break;
                     const int64_t o = row * P.N + col;
-                    if (P.mode == 3) atomicAdd((unsigned long long *)(P.partial + (int64_t)party * P.M * P.N + o), acc[j]);
+                    if (P.mode == 3) atomicAdd((unsigned long long *)(P.partial + (int64_t)(party - P.party_base) * P.M * P.N + o), acc[j]);
                     else P.C[P.mode == 2 ? 0 : party][o] = acc[j];
                 }
             }
@@ -512,7 +513,7 @@ __global__ void __launch_bounds__(192, 1) tc_ring_gemm64_v2(const TcParams<uint6
                     case 0: P.C[party][o] = P.C[party][o] + h; break;
                     case 1: P.C[party][o] = trunc_share<T>(P.C[party][o] + h + P.Z[party][o], party, P.trunc); break;
                     case 2: P.C[0][o] = P.C[0][o] + h - P.Z[0][o]; break;
-                    default: atomicAdd((unsigned long long *)(P.partial + (int64_t)party * P.M * P.N + o), h);
+                    default: atomicAdd((unsigned long long *)(P.partial + (int64_t)(party - P.party_base) * P.M * P.N + o), h);
                     }
                 }
             }
@@ -527,8 +528,9 @@ template <typename T>
 __global__ void tc_finalize_kernel(const TcParams<T> P, int mode) {
     const int64_t total = P.M * P.N * P.nparty;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
-        const int party = (int)(i / (P.M * P.N));
-        const int64_t o = i - (int64_t)party * P.M * P.N;
+        const int slot = (int)(i / (P.M * P.N));
+        const int party = P.party_base + slot;
+        const int64_t o = i - (int64_t)slot * P.M * P.N;
         const T acc = P.partial[i];
         if (mode == 0) P.C[party][o] = acc;
         else if (mode == 1) P.C[party][o] = trunc_share<T>(acc + P.Z[party][o], party, P.trunc);
@@ -695,13 +697,13 @@ size_t tc_beaver_ws_bytes(int64_t M, int64_t K, int64_t N) {
 }
 
 template <typename T>
-psml_status tc_beaver_matmul(Ctx *c, const T *const A[2], const T *const B[2], const T *const U[2], const T *const V[2],
-                             const T *const Z[2], int64_t M, int64_t K, int64_t N, int flags, int trunc, T *const C[2],
-                             cudaStream_t s) {
+psml_status tc_beaver_matmul_ws(const T *const A[2], const T *const B[2], const T *const U[2], const T *const V[2],
+                                const T *const Z[2], int64_t M, int64_t K, int64_t N, int flags, int trunc,
+                                T *const C[2], void *ws, size_t ws_bytes, int sm_count, cudaStream_t s) {
     constexpr int l = 8 * (int)sizeof(T);
     using Cf = tc::Cfg<l>;
-    PSML_TRY(c->ensure_ws(tc_beaver_ws_bytes<T>(M, K, N)));
-    uint8_t *w = (uint8_t *)c->ws;
+    if (ws_bytes < tc_beaver_ws_bytes<T>(M, K, N)) return fail(PSML_ERR_NOMEM, "tcgen05 Beaver workspace too small");
+    uint8_t *w = (uint8_t *)ws;
     auto carve = [&](size_t bytes) { uint8_t *p = w; w += (bytes + 255) & ~(size_t)255; return p; };
     T *mE0 = (T *)carve(sizeof(T) * M * K), *mE1 = (T *)carve(sizeof(T) * M * K);
     T *mF0 = (T *)carve(sizeof(T) * K * N), *mF1 = (T *)carve(sizeof(T) * K * N);
@@ -744,8 +746,67 @@ psml_status tc_beaver_matmul(Ctx *c, const T *const A[2], const T *const B[2], c
     P.nkb_lo = P.nkb_hi = (int)(sj.j[0].k_pad / tc::BK);
     P.M = M; P.N = N; P.nparty = 2; P.mode = 1; P.trunc = trunc;
     P.C[0] = C[0]; P.C[1] = C[1]; P.Z[0] = Z[0]; P.Z[1] = Z[1];
-    return tc::launch_gemm<l>(P, sj.j[0].rows_pad, sj.j[3].rows_pad, partial, 2 * M * N, c->sm_count, s);
+    return tc::launch_gemm<l>(P, sj.j[0].rows_pad, sj.j[3].rows_pad, partial, 2 * M * N, sm_count, s);
 }
+
+template <typename T>
+psml_status tc_beaver_matmul(Ctx *c, const T *const A[2], const T *const B[2], const T *const U[2], const T *const V[2],
+                             const T *const Z[2], int64_t M, int64_t K, int64_t N, int flags, int trunc, T *const C[2],
+                             cudaStream_t s) {
+    PSML_TRY(c->ensure_ws(tc_beaver_ws_bytes<T>(M, K, N)));
+    return tc_beaver_matmul_ws<T>(A, B, U, V, Z, M, K, N, flags, trunc, C, c->ws, c->ws_bytes, c->sm_count, s);
+}
+
+// Split deployment, round 2 for ONE party: the split round opens E = E_send + E_recv and
+// F = F_send + F_recv while writing the limb planes of D'_i (= U_0, or E + U_1), E, F and V_i.
+template <int l>
+static psml_status open_matmul_one(Ctx *c, int party, const void *Es, const void *Er, const void *Fs, const void *Fr,
+                                   const void *U, const void *V, const void *Z, int64_t M, int64_t K, int64_t N,
+                                   int trunc, void *C, cudaStream_t s) {
+    using Cf = tc::Cfg<l>;
+    using T = typename Cf::T;
+    const int64_t ta = tc::tiled_bytes<l>(M, K, tc::BM), tb = tc::tiled_bytes<l>(N, K, Cf::BN);
+    const size_t need = (size_t)(2 * ta + 2 * tb + sizeof(T) * M * N + 2048);
+    PSML_TRY(c->ensure_ws(need));
+    uint8_t *w = (uint8_t *)c->ws;
+    auto carve = [&](size_t bytes) { uint8_t *p = w; w += (bytes + 255) & ~(size_t)255; return p; };
+    uint8_t *tD = carve(ta), *tE = carve(ta), *tF = carve(tb), *tV = carve(tb);
+    T *partial = (T *)carve(sizeof(T) * M * N);
+    tc::SplitJobs sj;
+    sj.j[0] = party == 0 ? tc::make_job<l>(U, nullptr, nullptr, tD, M, K, tc::BM, 0)
+                         : tc::make_job<l>(Es, Er, U, tD, M, K, tc::BM, 0);
+    sj.j[1] = tc::make_job<l>(Es, Er, nullptr, tE, M, K, tc::BM, 0);
+    sj.j[2] = tc::make_job<l>(Fs, Fr, nullptr, tF, N, K, Cf::BN, 1);
+    sj.j[3] = tc::make_job<l>(V, nullptr, nullptr, tV, N, K, Cf::BN, 1);
+    sj.count = 4;
+    {
+        ProfScope prof(PROF_TC, s, 0.0);
+        PSML_TRY(tc::launch_split<l>(sj, s));
+    }
+    tc::TcParams<T> P{};
+    P.A_lo[0] = P.A_lo[1] = tD; P.A_hi[0] = P.A_hi[1] = tE;
+    P.B_lo[0] = P.B_lo[1] = tF; P.B_hi[0] = P.B_hi[1] = tV;
+    P.a_stride_lo = P.a_stride_hi = sj.j[0].rows_pad * sj.j[0].k_pad;
+    P.b_stride_lo = P.b_stride_hi = sj.j[2].rows_pad * sj.j[2].k_pad;
+    P.nkb_lo = P.nkb_hi = (int)(sj.j[0].k_pad / tc::BK);
+    P.M = M; P.N = N; P.nparty = 1; P.party_base = party; P.mode = 1; P.trunc = trunc;
+    P.C[0] = P.C[1] = (T *)C; P.Z[0] = P.Z[1] = (const T *)Z;
+    return tc::launch_gemm<l>(P, sj.j[0].rows_pad, sj.j[2].rows_pad, partial, M * N, c->sm_count, s);
+}
+
+psml_status tc_open_matmul_one(Ctx *c, int l, int party, const void *Es, const void *Er, const void *Fs,
+                               const void *Fr, const void *U, const void *V, const void *Z, int64_t M, int64_t K,
+                               int64_t N, int trunc, void *C, cudaStream_t s) {
+    if (l == 64) return open_matmul_one<64>(c, party, Es, Er, Fs, Fr, U, V, Z, M, K, N, trunc, C, s);
+    return open_matmul_one<32>(c, party, Es, Er, Fs, Fr, U, V, Z, M, K, N, trunc, C, s);
+}
+
+template size_t tc_beaver_ws_bytes<uint64_t>(int64_t, int64_t, int64_t);
+template size_t tc_beaver_ws_bytes<uint32_t>(int64_t, int64_t, int64_t);
+template psml_status tc_beaver_matmul_ws<uint64_t>(const uint64_t *const[2], const uint64_t *const[2],
+                                                   const uint64_t *const[2], const uint64_t *const[2],
+                                                   const uint64_t *const[2], int64_t, int64_t, int64_t, int, int,
+                                                   uint64_t *const[2], void *, size_t, int, cudaStream_t);
 
 template psml_status tc_beaver_matmul<uint64_t>(Ctx *, const uint64_t *const[2], const uint64_t *const[2],
                                                 const uint64_t *const[2], const uint64_t *const[2],

@@ -213,7 +213,11 @@ static int64_t ws_need(psml_model_s *m) {
     int64_t w = 0;
     for (auto &it : m->items[0]) {
         switch (it.kind) {
-        case IT_MATRIX: w = std::max(w, beaver_ws_words<T>(it.M, it.K, it.N)); break;
+        case IT_MATRIX:
+            w = std::max(w, beaver_ws_words<T>(it.M, it.K, it.N));
+            if (m->ctx->use_tc(it.M, 2 * it.K, it.N))
+                w = std::max(w, (int64_t)(tc_beaver_ws_bytes<T>(it.M, it.K, it.N) + 7) / 8);
+            break;
         case IT_CONV_FWD: w = std::max(w, conv_ws_words<T>(m->B, m->g, 0, it.N)); break;
         case IT_CONV_GW: w = std::max(w, conv_ws_words<T>(m->B, m->g, 1, it.N)); break;
         case IT_HAD: w = std::max(w, 4 * it.n); break;
@@ -224,9 +228,12 @@ static int64_t ws_need(psml_model_s *m) {
 }
 
 static int64_t dws_need(psml_model_s *m) {
-    int64_t w = 1;   // dealer: split-K partials of the Z = U V GEMMs
-    for (auto &it : m->items[0])
+    int64_t w = 1;   // dealer: split-K partials of the Z = U V GEMMs (or the tcgen05 limb planes)
+    for (auto &it : m->items[0]) {
         if (it.kind != IT_HAD && it.kind != IT_MSB) w = std::max(w, it.M * it.N);
+        if (it.kind == IT_MATRIX && m->ctx->use_tc(it.M, it.K, it.N))
+            w = std::max(w, (int64_t)(tc_ring_gemm_ws_bytes(64, it.M, it.K, it.N) + 7) / 8);
+    }
     return w;
 }
 
@@ -257,6 +264,9 @@ static psml_status deal_item(psml_model_s *m, DealItem &it, uint32_t step, cudaS
     switch (it.kind) {
     case IT_MATRIX: {
         PSML_TRY(deal_prg(m, it, cid, s));
+        if (m->ctx->use_tc(it.M, it.K, it.N))
+            return tc_dealer_gemm(64, it.U.p[0], it.U.p[1], it.V.p[0], it.V.p[1], it.M, it.K, it.N, it.Z.p[0],
+                                  it.Z.p[1], m->dws, sizeof(T) * (size_t)m->dws_words, s);
         DealerOps<T> ops;   // Z_1 = (U_0 + U_1)(V_0 + V_1) - Z_0
         ops.U0 = it.U.p[0]; ops.U1 = it.U.p[1]; ops.V0 = it.V.p[0]; ops.V1 = it.V.p[1];
         ops.Z0 = it.Z.p[0]; ops.Z1 = it.Z.p[1];
@@ -301,6 +311,9 @@ static psml_status mm(psml_model_s *m, const T *const A[2], const T *const Bm[2]
                       int trunc, T *const C[2], cudaStream_t s) {
     DealItem *it = find_item(m, layer, op, 0);
     if (!it) return fail(PSML_ERR_STATE, "missing triplet");
+    if (m->ctx->use_tc(it->M, 2 * it->K, it->N))
+        return tc_beaver_matmul_ws<T>(A, Bm, it->U.cp(), it->V.cp(), it->Z.cp(), it->M, it->K, it->N, flags, trunc, C,
+                                      m->ws, sizeof(T) * (size_t)m->ws_words, m->ctx->sm_count, s);
     return beaver_matmul<T>(A, Bm, it->U.cp(), it->V.cp(), it->Z.cp(), it->M, it->K, it->N, flags, trunc, C, m->ws,
                             m->ws_words, s, m->ctx->sm_count);
 }
@@ -448,6 +461,7 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
             desc->cnn_hidden <= 0 || desc->cnn_classes <= 0)
             return fail(PSML_ERR_SHAPE, "bad CNN geometry (cout must be <= 16)");
         g.OH = g.H - g.k + 1; g.OW = g.W - g.k + 1;
+        g.coloff = nullptr;
         m->g = g;
         m->nl = 3;
         const int64_t flat = (int64_t)g.OH * g.OW * desc->cnn_cout;
@@ -487,6 +501,17 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
     PSML_TRY(balloc(mp, m->yhat, B * m->dims[m->nl]));
     PSML_TRY(balloc(mp, m->delta, B * maxw));
     PSML_TRY(balloc(mp, m->tmp, B * maxw));
+    if (m->d.kind == PSML_CNN) {   // im2col column offsets (ch, ky, kx) -> ch*H*W + ky*W + kx
+        const ConvGeom &g = m->g;
+        std::vector<int32_t> off((size_t)g.C * g.k * g.k);
+        for (int ch = 0; ch < g.C; ++ch)
+            for (int ky = 0; ky < g.k; ++ky)
+                for (int kx = 0; kx < g.k; ++kx) off[(ch * g.k + ky) * g.k + kx] = (ch * g.H + ky) * g.W + kx;
+        T *dev = nullptr;
+        PSML_TRY(dalloc(mp, &dev, (int64_t)(off.size() + 1) / 2));
+        PSML_CUDA_TRY(cudaMemcpy(dev, off.data(), sizeof(int32_t) * off.size(), cudaMemcpyHostToDevice));
+        m->g.coloff = (const int32_t *)dev;
+    }
     plan_items(mp);
     m->items[1] = m->items[0];
     PSML_TRY(alloc_items(mp, m->items[0]));

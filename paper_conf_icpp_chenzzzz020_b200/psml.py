@@ -66,6 +66,8 @@ _SIGS = {
     "psml_msb_dealer": (i32, [Ring, u64, u64, i64, P2, vp]),
     "psml_secure_matmul": (i32, [vp, P2, P2, P2, P2, P2, i64, i64, i64, i32, i32, P2, vp, vp]),
     "psml_secure_hadamard": (i32, [vp, P2, P2, P2, P2, P2, i64, i32, P2, vp]),
+    "psml_beaver_mask": (i32, [vp, i32, vp, vp, vp, vp, i64, i64, i64, i32, vp, vp, vp]),
+    "psml_beaver_open_matmul": (i32, [vp, i32, vp, vp, vp, vp, vp, vp, vp, i64, i64, i64, i32, vp, vp]),
     "psml_truncate": (i32, [Ring, i32, vp, i64, i32, vp]),
     "psml_secure_msb": (i32, [vp, P2, i64, P2, P2, vp, vp]),
     "psml_secure_relu": (i32, [vp, P2, i64, P2, P2, P2, P2, P2, vp, vp]),
@@ -289,6 +291,24 @@ def secure_matmul(ctx, A, B, U, V, Z, M, K, N, flags=0, trunc=0, out=None, trace
           M, K, N, flags, trunc, _pair(C), ctypes.byref(tr) if tr is not None else None,
           _stream(stream))
     return (C, tr_t) if trace else C
+
+
+def beaver_mask(ctx, party, A_i, B_i, U_i, V_i, M, K, N, flags=0, stream=None):
+    """Split deployment, round 1 of party `party`: returns its send buffers (E_i, F_i)."""
+    E = empty(0, ctx.l, (M, K))
+    F = empty(0, ctx.l, (K, N))
+    _call("psml_beaver_mask", ctx.handle, party, _ptr(A_i), _ptr(B_i), _ptr(U_i), _ptr(V_i), M, K, N,
+          flags, _ptr(E), _ptr(F), _stream(stream))
+    return E, F
+
+
+def beaver_open_matmul(ctx, party, E_send, E_recv, F_send, F_recv, U_i, V_i, Z_i, M, K, N, trunc=0,
+                       out=None, stream=None):
+    """Split deployment, round 2 of party `party`: its share C_i of A.B (Eq. 8 shape)."""
+    C = out if out is not None else empty(0, ctx.l, (M, N))
+    _call("psml_beaver_open_matmul", ctx.handle, party, _ptr(E_send), _ptr(E_recv), _ptr(F_send),
+          _ptr(F_recv), _ptr(U_i), _ptr(V_i), _ptr(Z_i), M, K, N, trunc, _ptr(C), _stream(stream))
+    return C
 
 
 def secure_hadamard(ctx, A, B, U, V, Z, trunc=0, out=None, stream=None):
