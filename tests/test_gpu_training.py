@@ -98,3 +98,25 @@ def test_graph_replay_bitexact_vs_oracle(T, task, steps, pipelined):
         torch.cuda.synchronize()
         _compare_shares(tr, om)
     tr.close()
+
+
+def test_cnn_one_epoch_against_fp64(T):
+    """Config 4 (CIFAR-shaped CNN, 390 steps of 128): decoded master weights vs fp64 SGD."""
+    task = "cnn"
+    Wi = synth.init_weights(task)
+    tr = T.SecureTrainer(task, Wi, backend=0)
+    pm = plain.PlainModel(task, Wi)
+    steps = 50000 // 128
+    X, Y = synth.batch(task, 0)
+    tr.step(torch.from_numpy(X), torch.from_numpy(Y), 0)
+    pm.step(X, Y)
+    tr.capture(pipelined=True)
+    for s in range(1, steps):
+        X, Y = synth.batch(task, s)
+        tr.graph_step(torch.from_numpy(X), torch.from_numpy(Y), s)
+        pm.step(X, Y)
+    got = [w.cpu().numpy() for w in tr.master_weights()]
+    err = max(np.abs(g.reshape(w.shape) - w).max() for g, w in zip(got, pm.W))
+    print(f"cnn: one-epoch max |w - w_fp64| = 2^{np.log2(err):.2f}")
+    assert err < 2.0 ** -12
+    tr.close()
