@@ -463,6 +463,102 @@ __global__ void __launch_bounds__(256) msb_chain_fused_kernel(MsbArgs<T> a, Chai
     }
 }
 
+// ---- the whole chain in one launch, one LANE PER PARTY ------------------------------------------
+// Lanes 2i and 2i+1 run the same element for party 0 and party 1.  Each round a lane computes its
+// party's masked words, writes them to that party's send buffer (the transcript a split deployment
+// would exchange) and obtains the peer's words with a lane-pair shuffle -- the co-resident form
+// of the opening (Eq. 5 / boolean e = x ^ a).  G, P stay in registers.  MODE 0: msb, 1: ReLU,
+// 2: Eq. 9 (lanes 0-15 run 8 elements of the first half [z + 1/2], lanes 16-31 the matching
+// elements of the second half [z - 1/2]; the final difference is a shuffle by 16).
+template <typename T>
+__device__ __forceinline__ T peer_of(T v) {
+    return (T)__shfl_xor_sync(0xffffffffu, (unsigned long long)v, 1);
+}
+
+#define SEL(pair) (p ? (pair).p[1] : (pair).p[0])
+template <typename T, int MODE>
+__global__ void __launch_bounds__(256) msb_chain_pair_kernel(MsbArgs<T> a, ChainOut<T> o) {
+    constexpr int l = 8 * (int)sizeof(T);
+    constexpr int L = sizeof(T) == 8 ? 6 : 5;
+    const int lane = threadIdx.x & 31;
+    const int p = lane & 1;
+    const int64_t gtid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t n = a.n;
+    int64_t e;
+    bool valid, second = false;
+    if (MODE == 2) {
+        const int64_t nh = n >> 1;
+        const int64_t base = (gtid >> 5) * 8 + ((lane >> 1) & 7);
+        second = lane >= 16;
+        valid = base < nh;
+        e = valid ? (second ? base + nh : base) : 0;
+    } else {
+        e = gtid >> 1;
+        valid = e < n;
+        if (!valid) e = 0;
+    }
+    const T *mat = p ? a.mat.p[1] : a.mat.p[0];
+    T *msg = p ? a.msg.p[1] : a.msg.p[0];
+    auto M = [&](int t, int w) -> T { return mat[((int64_t)t * 3 + w) * n + e]; };
+    auto z_of = [&](T ee, T ff, int t) -> T {
+        T r = (ee & M(t, 1)) ^ (M(t, 0) & ff) ^ M(t, 2);
+        return p == 1 ? (T)(r ^ (ee & ff)) : r;
+    };
+    const T *xin = p ? a.x.p[1] : a.x.p[0];
+    const T half = p == 0 ? a.half : (T)0;
+    const T x = a.mode == 0 ? xin[e] : (e < (n >> 1) ? xin[e] + half : xin[e - (n >> 1)] - half);
+    // round 1: AND t = 0 on X = (x0, 0), Y = (0, x1)
+    T m0 = (p == 0 ? x : (T)0) ^ M(0, 0), m1 = (p == 1 ? x : (T)0) ^ M(0, 1);
+    if (valid) { msg[e] = m0; msg[n + e] = m1; }
+    T G = z_of(m0 ^ peer_of(m0), m1 ^ peer_of(m1), 0);
+    T P = x;
+#pragma unroll
+    for (int j = 1; j <= L; ++j) {
+        const int k = 1 << (j - 1);
+        const int t1 = 2 * j - 1, t2 = 2 * j;
+        const T g1 = P ^ M(t1, 0), h1 = (T)(G << k) ^ M(t1, 1);
+        T g2 = 0, h2 = 0;
+        if (j < L) { g2 = P ^ M(t2, 0); h2 = (T)(P << k) ^ M(t2, 1); }
+        if (valid) {
+            msg[e] = g1; msg[n + e] = h1;
+            if (j < L) { msg[2 * n + e] = g2; msg[3 * n + e] = h2; }
+        }
+        const T z1 = z_of(g1 ^ peer_of(g1), h1 ^ peer_of(h1), t1);
+        if (j < L) P = z_of(g2 ^ peer_of(g2), h2 ^ peer_of(h2), t2);
+        G ^= z1;
+    }
+    const T bit = ((x >> (l - 1)) & 1) ^ ((G >> (l - 2)) & 1);
+    if (valid && SEL(o.msbB)) SEL(o.msbB)[e] = bit;
+    const int64_t off = (int64_t)2 * L * 3 * n;
+    const T cm = bit ^ mat[off + e];          // B2A: c_i = msb_i ^ rB_i
+    if (valid) msg[e] = cm;
+    const T c = cm ^ peer_of(cm);
+    const T mA = (p == 0 ? c : (T)0) + ((T)1 - (T)2 * c) * mat[off + n + e];
+    if (MODE == 0) {
+        if (valid) SEL(o.msbA)[e] = mA;
+        return;
+    }
+    const T d = (p == 0 ? (T)1 : (T)0) - mA;  // DReLU share
+    if (valid && SEL(o.drelu)) SEL(o.drelu)[e] = d;
+    const T u = SEL(o.U)[e], v = SEL(o.V)[e];
+    const T me = x - u, mf = d - v;           // Hadamard round: mask
+    if (valid) { SEL(o.mE)[e] = me; SEL(o.mF)[e] = mf; }
+    const T E = me + peer_of(me), F = mf + peer_of(mf);
+    const T r = (T)p * E * F + E * v + u * F + SEL(o.Z)[e];
+    if (MODE == 1) {
+        if (valid) SEL(o.y)[e] = r;
+        return;
+    }
+    const T r2 = (T)__shfl_xor_sync(0xffffffffu, (unsigned long long)r, 16);
+    if (valid && !second) {
+        const T out = r - r2;                 // ReLU(z + 1/2) - ReLU(z - 1/2)
+        if (SEL(o.y)) SEL(o.y)[e] = out;
+        if (SEL(o.delta)) SEL(o.delta)[e] = out - SEL(o.Ysub)[e];
+    }
+}
+
+#undef SEL
+
 // ---------------------------------------------------------------------------------------------
 // training helpers
 // ---------------------------------------------------------------------------------------------

@@ -181,9 +181,12 @@ psml_status msb_chain(const T *const x[2], int64_t n, const T *const mat[2], int
     o.mE = mE;
     o.mF = mF;
     o.what = what;
-    if (chain_mode() == 0) {   // all rounds of an element in one thread, one launch
-        const int64_t units = what == 2 ? n / 2 : n;
-        msb_chain_fused_kernel<T><<<ew_grid(units), EW_THREADS, 0, s>>>(a, o);
+    if (chain_mode() == 0) {   // one launch; lane pair = (party 0, party 1) of one element
+        const int64_t threads = what == 2 ? ((n / 2 + 7) / 8) * 32 : 2 * n;
+        const int blocks = (int)((threads + EW_THREADS - 1) / EW_THREADS);
+        if (what == 0) msb_chain_pair_kernel<T, 0><<<blocks, EW_THREADS, 0, s>>>(a, o);
+        else if (what == 1) msb_chain_pair_kernel<T, 1><<<blocks, EW_THREADS, 0, s>>>(a, o);
+        else msb_chain_pair_kernel<T, 2><<<blocks, EW_THREADS, 0, s>>>(a, o);
         PSML_LAUNCH_CHECK();
         return PSML_OK;
     }
