@@ -89,6 +89,47 @@ struct BeaverOps {
     }
 };
 
+// Co-resident Beaver product with the mask round fused into the operand loads: the opened
+// E = (op(A)_0 - U_0) + (op(A)_1 - U_1) and F likewise are formed where the GEMM reads them (the
+// same ring arithmetic as mask kernel + open; no message buffers, one launch less per product).
+// a_kmajor()/b_kmajor() tell the loaders which index is contiguous so transposed operands stay
+// coalesced.
+template <typename T>
+struct BeaverFusedOps {
+    const T *A[2], *B[2], *U[2], *V[2], *Z[2];
+    T *C[2];
+    int64_t M, N, K, Kext;
+    int transA, transB, trunc;
+    static constexpr int nparty = 2;
+    __device__ __forceinline__ bool a_kmajor() const { return !transA; }
+    __device__ __forceinline__ bool b_nmajor() const { return !transB; }
+    __device__ __forceinline__ T opA(int p, int64_t m, int64_t k) const {
+        return transA ? A[p][k * M + m] : A[p][m * K + k];
+    }
+    __device__ __forceinline__ T opB(int p, int64_t k, int64_t n) const {
+        return transB ? B[p][n * K + k] : B[p][k * N + n];
+    }
+    __device__ __forceinline__ T a(int p, int64_t m, int64_t k) const {
+        const bool first = k < K;
+        if (!first) k -= K;
+        const int64_t u = m * K + k;
+        const T e = (opA(0, m, k) - U[0][u]) + (opA(1, m, k) - U[1][u]);
+        return first ? (T)((T)p * e + U[p][u]) : e;
+    }
+    __device__ __forceinline__ T b(int p, int64_t k, int64_t n) const {
+        if (k < K) return (opB(0, k, n) - V[0][k * N + n]) + (opB(1, k, n) - V[1][k * N + n]);
+        return V[p][(k - K) * N + n];
+    }
+    __device__ __forceinline__ void store(int p, int64_t m, int64_t n, T acc) const {
+        C[p][m * N + n] = trunc_share<T>(acc + Z[p][m * N + n], p, trunc);
+    }
+};
+
+template <class Ops> __device__ __forceinline__ bool ops_a_kmajor(const Ops &o, int) { return true; }
+template <class Ops> __device__ __forceinline__ bool ops_b_nmajor(const Ops &o, int) { return true; }
+template <typename T> __device__ __forceinline__ bool ops_a_kmajor(const BeaverFusedOps<T> &o, int) { return o.a_kmajor(); }
+template <typename T> __device__ __forceinline__ bool ops_b_nmajor(const BeaverFusedOps<T> &o, int) { return o.b_nmajor(); }
+
 // One party of the split deployment: own messages (mE0/mF0 = sent) + the peer's (mE1/mF1 =
 // received); same arithmetic as BeaverOps for party `party`.
 template <typename T>
@@ -318,14 +359,24 @@ __global__ void __launch_bounds__(256) ring_gemm_small(Ops ops, int64_t k_per_sp
     const int tid = threadIdx.x;
     const int tx = tid & 15, ty = tid >> 4;
     T ra[4], rb[4];
+    // thread -> element maps: A 16 x 64 consecutive along k (row-major A) or along m (A^T);
+    // B 64 x 16 consecutive along n (row-major B) or along k (B^T)
+    const bool ak = ops_a_kmajor(ops, 0), bn = ops_b_nmajor(ops, 0);
+    auto amap = [&](int idx, int &mm, int &kk) {
+        if (ak) { mm = idx >> 6; kk = idx & 63; } else { mm = idx & 15; kk = idx >> 4; }
+    };
+    auto bmap = [&](int idx, int &kb, int &nn) {
+        if (bn) { kb = idx >> 4; nn = idx & 15; } else { kb = idx & 63; nn = idx >> 6; }
+    };
     auto load = [&](int64_t k0) {
 #pragma unroll
         for (int t = 0; t < 4; ++t) {
             const int idx = tid + t * 256;
-            const int mm = idx >> 6, kk = idx & 63;          // A: 16 x 64, coalesced along k
+            int mm, kk, kb, nn;
+            amap(idx, mm, kk);
             const int64_t m = m0 + mm, k = k0 + kk;
             ra[t] = (m < ops.M && k < kend) ? ops.a(p, m, k) : (T)0;
-            const int kb = idx >> 4, nn = idx & 15;          // B: 64 x 16, coalesced along n
+            bmap(idx, kb, nn);
             const int64_t k2 = k0 + kb, n = n0 + nn;
             rb[t] = (n < ops.N && k2 < kend) ? ops.b(p, k2, n) : (T)0;
         }
@@ -334,8 +385,11 @@ __global__ void __launch_bounds__(256) ring_gemm_small(Ops ops, int64_t k_per_sp
 #pragma unroll
         for (int t = 0; t < 4; ++t) {
             const int idx = tid + t * 256;
-            As[buf][idx >> 6][idx & 63] = ra[t];
-            Bs[buf][idx >> 4][idx & 15] = rb[t];
+            int mm, kk, kb, nn;
+            amap(idx, mm, kk);
+            bmap(idx, kb, nn);
+            As[buf][mm][kk] = ra[t];
+            Bs[buf][kb][nn] = rb[t];
         }
     };
     T acc = 0;

@@ -84,6 +84,24 @@ psml_status beaver_matmul(const T *const A[2], const T *const B[2], const T *con
     return PSML_OK;
 }
 
+// Co-resident Beaver matmul with the mask round fused into the GEMM's operand loads (one launch;
+// bit-identical to beaver_matmul).  ws: 2*M*N words for split-K partials.
+template <typename T>
+psml_status beaver_matmul_fused(const T *const A[2], const T *const B[2], const T *const U[2],
+                                const T *const V[2], const T *const Z[2], int64_t M, int64_t K,
+                                int64_t N, int flags, int trunc, T *const C[2], T *ws, int64_t ws_words,
+                                cudaStream_t s, int sm_count) {
+    BeaverFusedOps<T> ops;
+    for (int p = 0; p < 2; ++p) {
+        ops.A[p] = A[p]; ops.B[p] = B[p]; ops.U[p] = U[p]; ops.V[p] = V[p]; ops.Z[p] = Z[p]; ops.C[p] = C[p];
+    }
+    ops.M = M; ops.N = N; ops.K = K; ops.Kext = 2 * K;
+    ops.transA = (flags & PSML_TRANS_A) ? 1 : 0;
+    ops.transB = (flags & PSML_TRANS_B) ? 1 : 0;
+    ops.trunc = trunc;
+    return launch_ring_gemm<T, BeaverFusedOps<T>>(ops, ws, ws_words, s, sm_count);
+}
+
 // ---------------------------------------------------------------------------------------------
 // Convolution Beaver product (im2col ring GEMM, mask on the raw input; R17)
 // transposed = 0: C = im2col(X) . Wc         M = B*OH*OW, K = C*k*k,  N = Cout

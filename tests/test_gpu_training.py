@@ -120,3 +120,17 @@ def test_cnn_one_epoch_against_fp64(T):
     print(f"cnn: one-epoch max |w - w_fp64| = 2^{np.log2(err):.2f}")
     assert err < 2.0 ** -12
     tr.close()
+
+
+def test_explicit_mask_round_matches_fused_open():
+    """PSML_OPEN=fused (mask round fused into the GEMM loads) and PSML_MSB_CHAIN=rounds (one
+    kernel per protocol round) reproduce the oracle exactly, like the defaults."""
+    import os
+    import subprocess
+    import sys
+    env = dict(os.environ, PSML_OPEN="fused", PSML_MSB_CHAIN="rounds")
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu", "-k",
+                        "training_bitexact_vs_oracle", os.path.join(root, "tests", "test_gpu_training.py")],
+                       env=env, capture_output=True, text=True, cwd=root)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
