@@ -122,9 +122,17 @@ def dist_setup(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # PSML_DIST_BACKEND=gloo + PSML_SHARE_GPU=1: all ranks on cuda:0 over gloo -- exercises the
+    # data-parallel path on a one-GPU box (not a performance configuration).
+    backend = os.environ.get("PSML_DIST_BACKEND", "nccl")
+    if os.environ.get("PSML_SHARE_GPU") == "1":
+        local = 0
     if world > 1:
         torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
     else:
         torch.cuda.set_device(0)
     return world, rank, local

@@ -77,3 +77,97 @@ def split_secure_matmul(ctx, party, A_i, B_i, U_i, V_i, Z_i, M, K, N, flags=0, t
     E, F = psml.beaver_mask(ctx, party, A_i, B_i, U_i, V_i, M, K, N, flags)
     Er, Fr = exchange([E, F], peer, group)
     return psml.beaver_open_matmul(ctx, party, E, Er, F, Fr, U_i, V_i, Z_i, M, K, N, trunc)
+
+
+class CompressedChannel:
+    """Compressed transmission of PAPER.md Sec. 4.4 (Eqs. 10-12) for the split deployment.
+
+    Each message slot remembers the last message it sent and received.  The next message of the
+    slot is sent as its delta against the previous one (E_{i,j+1} = E_{i,j} + Delta, Eq. 11), in
+    CSR form when >= 75% of the delta is zero (psml_delta_encode) and dense otherwise; the receiver
+    rebuilds the peer's message with psml_delta_apply.  The first message of a slot is dense.
+    Two exchanges per compressed message: an 8-word header (format, nnz), then the payload.
+    (With fresh masks per step the delta of a masked message is uniformly random -- dense; only a
+    constant operand under a persistent mask gives an empty CSR, R19.)
+    """
+
+    def __init__(self, ctx, peer, group=None):
+        self.ctx, self.peer, self.group = ctx, peer, group
+        self.prev_send, self.prev_recv = {}, {}
+        self.bytes_sent = 0
+        self.formats = []
+
+    def _words(self, t):
+        return t.view(torch.int64) if t.dtype == torch.uint64 else t.view(torch.int32)
+
+    def exchange(self, key, t):
+        from . import psml
+        if t.dim() != 2:
+            raise ValueError("messages are matrices (rows x cols)")
+        prev = self.prev_send.get(key)
+        if prev is None:
+            (r,) = exchange([t], self.peer, self.group)
+            self.bytes_sent += t.numel() * t.element_size()
+            self.formats.append("dense-first")
+        else:
+            enc = psml.delta_encode(self.ctx, t, prev)
+            rows, cols = t.shape
+            hdr = torch.tensor([1 if enc["is_csr"] else 0, enc["nnz"], rows, cols, 0, 0, 0, 0],
+                               dtype=torch.int64, device=t.device)
+            (phdr,) = exchange([hdr], self.peer, self.group)
+            p_csr, p_nnz = int(phdr[0]), int(phdr[1])
+            if enc["is_csr"]:
+                send = [enc["row_ptr"]] + ([enc["col_idx"], enc["vals"]] if enc["nnz"] else [])
+                self.bytes_sent += 64 + sum(x.numel() * x.element_size() for x in send)
+            else:
+                send = [enc["dense"]]
+                self.bytes_sent += 64 + t.numel() * t.element_size()
+            self.formats.append("csr" if enc["is_csr"] else "dense")
+            # receive the peer's payload (shapes known from its header)
+            if p_csr:
+                recv_like = [torch.empty(rows + 1, dtype=torch.int32, device=t.device)]
+                if p_nnz:
+                    recv_like += [torch.empty(p_nnz, dtype=torch.int32, device=t.device),
+                                  torch.empty(p_nnz, dtype=t.dtype, device=t.device)]
+            else:
+                recv_like = [torch.empty_like(t)]
+            got = _exchange_uneven(send, recv_like, self.peer, self.group)
+            r = self.prev_recv[key].clone()
+            if p_csr:
+                penc = dict(is_csr=True, nnz=p_nnz, row_ptr=got[0],
+                            col_idx=got[1] if p_nnz else None, vals=got[2] if p_nnz else None)
+            else:
+                penc = dict(is_csr=False, nnz=p_nnz, dense=got[0])
+            psml.delta_apply(self.ctx, r, penc)
+        self.prev_send[key] = t.clone()
+        self.prev_recv[key] = r.clone()
+        return r
+
+
+def _exchange_uneven(send, recv_like, peer, group=None):
+    """Send the tensors `send` and receive tensors shaped like `recv_like` (may differ)."""
+    import torch.distributed as dist
+    stage = dist.get_backend(group) != "nccl"
+    cast = lambda t: t.view(torch.int64) if t.dtype == torch.uint64 else (  # noqa: E731
+        t.view(torch.int32) if t.dtype == torch.uint32 else t)
+    ops, dst = [], []
+    for t in send:
+        src = cast(t)
+        ops.append(dist.P2POp(dist.isend, src.cpu() if stage else src, peer, group))
+    for t in recv_like:
+        d = torch.empty_like(cast(t), device="cpu") if stage else torch.empty_like(cast(t))
+        ops.append(dist.P2POp(dist.irecv, d, peer, group))
+        dst.append((t, d))
+    for req in dist.batch_isend_irecv(ops):
+        req.wait()
+    return [(d.to(t.device) if stage else d).view(t.dtype) for t, d in dst]
+
+
+def split_secure_matmul_compressed(ctx, channel, slot, party, A_i, B_i, U_i, V_i, Z_i, M, K, N,
+                                   flags=0, trunc=0):
+    """split_secure_matmul with the opening sent through a CompressedChannel (slot = message id)."""
+    from . import psml
+    E, F = psml.beaver_mask(ctx, party, A_i, B_i, U_i, V_i, M, K, N, flags)
+    Er = channel.exchange((slot, "E"), E)
+    Fr = channel.exchange((slot, "F"), F)
+    return psml.beaver_open_matmul(ctx, party, E, Er, F, Fr, U_i, V_i, Z_i, M, K, N, trunc)
