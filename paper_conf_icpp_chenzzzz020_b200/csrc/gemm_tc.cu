@@ -192,6 +192,7 @@ struct TcParams {
     const T *Z[2];
     int trunc;
     T *partial;        // mode 3: nparty x M x N
+    int debug;         // experiments only (PSML_TC_DEBUG): 1 = skip pass-H stores, 2 = skip pass-L stores
 };
 
 // Epilogue chunk: thread `lane` holds 16 consecutive columns of row row0 + lane (the TMEM 32x32b
@@ -476,7 +477,7 @@ __global__ void __launch_bounds__(192, 1) tc_ring_gemm64_v2(const TcParams<uint6
                 tc_fence_before();
                 mbar_arrive(smem_u32(acce));
             }
-            if (row < P.M) {
+            if (row < P.M && !(P.debug & 2)) {
 #pragma unroll
                 for (int j = 0; j < 16; ++j) {
                     const int64_t col = col0 + j0 + j;
@@ -504,7 +505,7 @@ __global__ void __launch_bounds__(192, 1) tc_ring_gemm64_v2(const TcParams<uint6
 #pragma unroll
                 for (int j = 0; j < 16; ++j) hi[j] += r[j] << (8 * s);
             }
-            if (row < P.M) {
+            if (row < P.M && !(P.debug & 1)) {
 #pragma unroll
                 for (int j = 0; j < 16; ++j) {
                     const int64_t col = col0 + j0 + j;
@@ -571,6 +572,203 @@ __device__ __forceinline__ void tc_commit_2sm(uint32_t bar) {
         "}\n" ::"r"(bar)
         : "memory");
 }
+
+// ------------------------------------------------------------------------------------------------
+// l = 64, v4: v2 with the passes reversed and the high half kept ON CHIP.
+//   pass H first (shifts 4..7, 26 limb pairs): the epilogue warps fold the 4 accumulators into
+//   high = sum S_s 2^{8(s-4)} mod 2^32 and park it in shared memory (128 x 128 x 4 B = 64 KB);
+//   pass L (shifts 0..3, 10 limb pairs): the epilogue forms low + high 2^32 and stores C once.
+// v2 staged the 64-bit pass-L partial through HBM (store + reload): measured 9-12% of the kernel.
+// The 128 KB pipeline region is re-partitioned between passes: 2 x 64 KB stages in pass H
+// (8 limbs of A and B per 32-byte K block), 4 x 32 KB stages in pass L (4 limbs each).
+// ------------------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(192, 1) tc_ring_gemm64_v4(const TcParams<uint64_t> P) {
+    using T = uint64_t;
+    constexpr int BN = 128, L = 8;
+    constexpr int A_BYTES = BM * BK, B_BYTES = BN * BK;
+    constexpr int REGION = 2 * L * (A_BYTES + B_BYTES);               // 128 KB
+    constexpr int SH_BYTES = L * (A_BYTES + B_BYTES), SL_BYTES = 4 * (A_BYTES + B_BYTES);
+    constexpr uint32_t IDESC = idesc_i8(BM, BN);
+    extern __shared__ __align__(1024) uint8_t smem[];
+    uint32_t *hi_buf = (uint32_t *)(smem + REGION);                   // [col][row]
+    uint64_t *bars = (uint64_t *)(smem + REGION + BM * BN * 4);
+    uint64_t *fullH = bars, *emptyH = bars + 2, *fullL = bars + 4, *emptyL = bars + 8;
+    uint64_t *accf = bars + 12, *acce = bars + 13;
+    uint32_t *tmem_slot = (uint32_t *)(bars + 14);
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int party = P.party_base + blockIdx.z % P.nparty, split = blockIdx.z / P.nparty;
+    const int nb = blockIdx.x, rb = blockIdx.y;
+    const int nkb = P.nkb_lo + P.nkb_hi;
+    const int kb0 = split * P.kb_per_split;
+    const int kb1 = min(kb0 + P.kb_per_split, nkb);
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < 2; ++s) { mbar_init(smem_u32(&fullH[s]), 1); mbar_init(smem_u32(&emptyH[s]), 1); }
+        for (int s = 0; s < 4; ++s) { mbar_init(smem_u32(&fullL[s]), 1); mbar_init(smem_u32(&emptyL[s]), 1); }
+        mbar_init(smem_u32(accf), 1);
+        mbar_init(smem_u32(acce), 128);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if (warp == 2) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_u32(tmem_slot)));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem = *tmem_slot;
+
+    auto tile_src = [&](int kb, const uint8_t *&a, const uint8_t *&b, int64_t &as, int64_t &bs) {
+        const bool lo = kb < P.nkb_lo;
+        const int kk = lo ? kb : kb - P.nkb_lo;
+        const int nk = lo ? P.nkb_lo : P.nkb_hi;
+        a = (lo ? P.A_lo[party] : P.A_hi[party]) + ((int64_t)rb * nk + kk) * A_BYTES;
+        b = (lo ? P.B_lo[party] : P.B_hi[party]) + ((int64_t)nb * nk + kk) * B_BYTES;
+        as = lo ? P.a_stride_lo : P.a_stride_hi;
+        bs = lo ? P.b_stride_lo : P.b_stride_hi;
+    };
+
+    if (warp == 0) {
+        if (lane == 0) {
+            // ---------------- producer: pass H (2 x 64 KB), then pass L (4 x 32 KB) ----------------
+            int st = 0;
+            uint32_t ph = 0;
+            for (int kb = kb0; kb < kb1; ++kb) {
+                mbar_wait(smem_u32(&emptyH[st]), ph ^ 1);
+                const uint32_t fb = smem_u32(&fullH[st]);
+                mbar_expect_tx(fb, (uint32_t)SH_BYTES);
+                const uint8_t *a, *b;
+                int64_t as, bs;
+                tile_src(kb, a, b, as, bs);
+                uint8_t *sa = smem + st * SH_BYTES, *sb = sa + L * A_BYTES;
+                for (int q = 0; q < L; ++q) bulk_g2s(smem_u32(sa + q * A_BYTES), a + q * as, A_BYTES, fb);
+                for (int q = 0; q < L; ++q) bulk_g2s(smem_u32(sb + q * B_BYTES), b + q * bs, B_BYTES, fb);
+                if (++st == 2) { st = 0; ph ^= 1; }
+            }
+            for (int i = 0; i < 2; ++i) {   // both pass-H slots consumed before re-partitioning
+                mbar_wait(smem_u32(&emptyH[st]), ph ^ 1);
+                if (++st == 2) { st = 0; ph ^= 1; }
+            }
+            st = 0;
+            ph = 0;
+            for (int kb = kb0; kb < kb1; ++kb) {
+                mbar_wait(smem_u32(&emptyL[st]), ph ^ 1);
+                const uint32_t fb = smem_u32(&fullL[st]);
+                mbar_expect_tx(fb, (uint32_t)SL_BYTES);
+                const uint8_t *a, *b;
+                int64_t as, bs;
+                tile_src(kb, a, b, as, bs);
+                uint8_t *sa = smem + st * SL_BYTES, *sb = sa + 4 * A_BYTES;
+                for (int q = 0; q < 4; ++q) bulk_g2s(smem_u32(sa + q * A_BYTES), a + q * as, A_BYTES, fb);
+                for (int q = 0; q < 4; ++q) bulk_g2s(smem_u32(sb + q * B_BYTES), b + q * bs, B_BYTES, fb);
+                if (++st == 4) { st = 0; ph ^= 1; }
+            }
+        }
+    } else if (warp == 1) {
+        if (lane == 0) {
+            // ---------------- MMA issuer ----------------
+            int st = 0;
+            uint32_t ph = 0;
+            for (int kb = kb0; kb < kb1; ++kb) {   // pass H: shifts 4..7
+                mbar_wait(smem_u32(&fullH[st]), ph);
+                tc_fence_after();
+                const uint32_t sa = smem_u32(smem + st * SH_BYTES), sb = sa + L * A_BYTES;
+#pragma unroll
+                for (int p = 0; p < 8; ++p) {
+                    const uint64_t ad = smem_desc(sa + p * A_BYTES, 128, 256);
+#pragma unroll
+                    for (int q = (p < 4 ? 4 - p : 0); q < 8 - p; ++q)
+                        tc_mma_i8(tmem + (uint32_t)((p + q - 4) * BN), ad, smem_desc(sb + q * B_BYTES, 128, 256), IDESC,
+                                  (kb > kb0 || p > 0) ? 1u : 0u);
+                }
+                tc_commit(smem_u32(&emptyH[st]));
+                if (++st == 2) { st = 0; ph ^= 1; }
+            }
+            tc_commit(smem_u32(accf));
+            mbar_wait(smem_u32(acce), 0);           // high half parked in smem, TMEM free
+            tc_fence_after();
+            st = 0;
+            ph = 0;
+            for (int kb = kb0; kb < kb1; ++kb) {   // pass L: shifts 0..3
+                mbar_wait(smem_u32(&fullL[st]), ph);
+                tc_fence_after();
+                const uint32_t sa = smem_u32(smem + st * SL_BYTES), sb = sa + 4 * A_BYTES;
+#pragma unroll
+                for (int p = 0; p < 4; ++p) {
+                    const uint64_t ad = smem_desc(sa + p * A_BYTES, 128, 256);
+#pragma unroll
+                    for (int q = 0; q < 4 - p; ++q)
+                        tc_mma_i8(tmem + (uint32_t)((p + q) * BN), ad, smem_desc(sb + q * B_BYTES, 128, 256), IDESC,
+                                  (kb > kb0 || p > 0) ? 1u : 0u);
+                }
+                tc_commit(smem_u32(&emptyL[st]));
+                if (++st == 4) { st = 0; ph ^= 1; }
+            }
+            tc_commit(smem_u32(accf));
+        }
+    } else {
+        // ---------------- epilogue warps 2..5 ----------------
+        const int quarter = warp & 3;
+        const int rl = quarter * 32 + lane;                 // row within the tile
+        const int64_t row = (int64_t)rb * BM + rl;
+        const uint32_t lane_base = tmem + ((uint32_t)(quarter * 32) << 16);
+        const int64_t col0 = (int64_t)nb * BN;
+        mbar_wait(smem_u32(accf), 0);
+        tc_fence_after();
+#pragma unroll 1
+        for (int j0 = 0; j0 < BN; j0 += 16) {
+            uint32_t hi[16];
+#pragma unroll
+            for (int j = 0; j < 16; ++j) hi[j] = 0;
+#pragma unroll
+            for (int s = 0; s < 4; ++s) {
+                uint32_t r[16];
+                tmem_ld16(lane_base + (uint32_t)(s * BN + j0), r);
+#pragma unroll
+                for (int j = 0; j < 16; ++j) hi[j] += r[j] << (8 * s);
+            }
+#pragma unroll
+            for (int j = 0; j < 16; ++j) hi_buf[(j0 + j) * BM + rl] = hi[j];
+        }
+        tc_fence_before();
+        mbar_arrive(smem_u32(acce));
+        mbar_wait(smem_u32(accf), 1);
+        tc_fence_after();
+#pragma unroll 1
+        for (int j0 = 0; j0 < BN; j0 += 16) {
+            T acc[16];
+#pragma unroll
+            for (int j = 0; j < 16; ++j) acc[j] = (T)hi_buf[(j0 + j) * BM + rl] << 32;
+#pragma unroll
+            for (int s = 0; s < 4; ++s) {
+                uint32_t r[16];
+                tmem_ld16(lane_base + (uint32_t)(s * BN + j0), r);
+#pragma unroll
+                for (int j = 0; j < 16; ++j) acc[j] += (T)r[j] << (8 * s);
+            }
+            if (row < P.M && !(P.debug & 1)) {
+#pragma unroll
+                for (int j = 0; j < 16; ++j) {
+                    const int64_t col = col0 + j0 + j;
+                    if (col >= P.N) break;
+                    const int64_t o = row * P.N + col;
+                    switch (P.mode) {
+                    case 0: P.C[party][o] = acc[j]; break;
+                    case 1: P.C[party][o] = trunc_share<T>(acc[j] + P.Z[party][o], party, P.trunc); break;
+                    case 2: P.C[0][o] = acc[j] - P.Z[0][o]; break;
+                    default: atomicAdd((unsigned long long *)(P.partial + (int64_t)(party - P.party_base) * P.M * P.N + o), acc[j]);
+                    }
+                }
+            }
+        }
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 2) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tmem));
+}
+
+constexpr size_t smem_v4_bytes() { return (size_t)2 * 8 * (BM * BK + 128 * BK) + (size_t)BM * 128 * 4 + 16 * 8; }
 
 template <int STAGES>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(192, 1) tc_ring_gemm64_2sm(const TcParams<uint64_t> P) {
@@ -832,6 +1030,8 @@ static psml_status launch_gemm(TcParams<typename Cfg<l>::T> P, int64_t Mp, int64
     int kbs = (nkb + splits - 1) / splits;
     splits = (nkb + kbs - 1) / kbs;
     P.kb_per_split = kbs;
+    static const int dbg = getenv("PSML_TC_DEBUG") ? atoi(getenv("PSML_TC_DEBUG")) : 0;
+    P.debug = dbg;
     const int final_mode = P.mode;
     if (splits > 1) {
         if (!partial || partial_words < P.M * P.N * P.nparty)
@@ -854,7 +1054,7 @@ static psml_status launch_gemm(TcParams<typename Cfg<l>::T> P, int64_t Mp, int64
                 }
                 dim3 g2((unsigned)(2 * (Np / BN)), (unsigned)(Mp / (2 * BM)), grid.z);   // x = (n tile, pair rank)
                 kern<<<g2, 192, smem_pair_bytes(), s>>>(P);
-            } else {
+            } else if (getenv("PSML_TC_V2")) {   // previous schedule (pass-L partial via HBM)
                 auto kern = tc_ring_gemm64_v2<Cfg<l>::STAGES>;
                 static bool attr_set = false;
                 if (!attr_set) {
@@ -862,6 +1062,14 @@ static psml_status launch_gemm(TcParams<typename Cfg<l>::T> P, int64_t Mp, int64
                     attr_set = true;
                 }
                 kern<<<grid, 192, smem_bytes<l>(), s>>>(P);
+            } else {
+                auto kern = tc_ring_gemm64_v4;
+                static bool attr_set = false;
+                if (!attr_set) {
+                    PSML_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_v4_bytes()));
+                    attr_set = true;
+                }
+                kern<<<grid, 192, smem_v4_bytes(), s>>>(P);
             }
         } else {
             auto kern = tc_ring_gemm_kernel<T, Cfg<l>::L, BN, Cfg<l>::STAGES>;
