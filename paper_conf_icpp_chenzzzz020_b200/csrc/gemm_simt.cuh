@@ -491,7 +491,7 @@ psml_status launch_ring_gemm(const Ops &ops, T *ws, int64_t ws_words, cudaStream
     // kernel choice: warp-per-row GEMV for skinny outputs with few rows (w^T x, MLP output layer),
     // the 16 x 16 small-tile kernel for small outputs or skinny outputs with many rows (CNN conv
     // im2col GEMMs), the 64 x 64 register-blocked kernel otherwise.
-    const bool gemv = N <= 16 && M * Ops::nparty <= 4096 && Kx <= 8192;
+    const bool gemv = N <= 2 && M * Ops::nparty <= 4096 && Kx <= 8192;
     const bool small = !gemv && (N <= 16 || M * N * Ops::nparty <= ((int64_t)1 << 18));
     int splits = 1;
     if (small) {
