@@ -225,6 +225,23 @@ def bench_ours(args):
     launches = psml.kernel_launch_count() - l0
     t_dev = max_over_ranks(t_dev, world)
 
+    # online-only CUDA graph (diagnostic): re-capture the step without the dealer branch and
+    # replay it on material dealt once (timing only -- a real run never reuses triplets)
+    t_on_graph = None
+    if world == 1:
+        tr.model.deal(0)
+        gs = torch.cuda.Stream()
+        gs.wait_stream(stream)
+        with torch.cuda.stream(gs):
+            tr.model.capture_step(tr.Xbuf, tr.Ybuf, with_deal=False, with_update=True, pipelined=False,
+                                  stream=gs)
+        stream.wait_stream(gs)
+        tr.model.step_graph(0)
+        torch.cuda.synchronize()
+        t_on_graph = timed(lambda s: tr.model.step_graph(0), K, 0)
+        tr.capture(with_update=True)   # restore the pipelined graph for the e2e leg
+        tr._next_dealt = None
+
     # online-only (dealer material generated before each step, outside the events)
     evs = []
     for i in range(K):
@@ -268,6 +285,7 @@ def bench_ours(args):
                    "l2": "256 MiB flush between timed steps (outside the events)",
                    "step": "client encode+share, dealer (offline), online secure step"},
         "online_samples_per_s": samples / t_on,
+        "online_graph_samples_per_s": (samples / t_on_graph) if t_on_graph else None,
         "eager_samples_per_s": samples / t_eager,
         "cuda_graph": {"kernel_nodes_per_step": n_nodes,
                        "note": "value/e2e replay one captured graph per step (dealer + online "

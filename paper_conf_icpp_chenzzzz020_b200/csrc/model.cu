@@ -17,6 +17,7 @@
 #include <vector>
 
 #include "engine.h"
+#include "dealer_fused.cuh"
 
 namespace psml {
 
@@ -35,6 +36,17 @@ static bool fused_open() {
     if (m < 0) {
         const char *e = getenv("PSML_OPEN");
         m = (e && e[0] == 'f') ? 1 : 0;
+    }
+    return m == 1;
+}
+
+// The whole dealer of one step as two launches (dealer_fused.cuh; default) or one launch group per
+// item (PSML_DEAL=items); bit-identical (tested).
+static bool fused_deal() {
+    static int m = -1;
+    if (m < 0) {
+        const char *e = getenv("PSML_DEAL");
+        m = (e && e[0] == 'i') ? 0 : 1;
     }
     return m == 1;
 }
@@ -59,6 +71,16 @@ struct DealItem {
     Buf U, V, Z, mat;
 };
 
+struct DealPlan {   // fused dealer of one pool (full or inference-only)
+    PrgJob *prg = nullptr;
+    int n_prg = 0;
+    int64_t prg_blocks = 0;
+    GemmJob *gemm = nullptr;
+    int n_gemm = 0;
+    int64_t gemm_tiles = 0;
+    std::vector<int> rest;   // items whose Z = U V runs in its own launch (conv, tcgen05-sized)
+};
+
 }  // namespace psml
 
 struct psml_model_s {
@@ -79,6 +101,7 @@ struct psml_model_s {
     // Dealer pools, double-buffered: step s consumes pool s % 2, so the dealer of step s + 1 can
     // run concurrently with the online phase of step s (offline/online pipelining).
     std::vector<psml::DealItem> items[2];
+    psml::DealPlan plan[2][2];         // [pool][infer_only]
     int pool = 0;                      // pool the online phase is reading
     psml::T *ws = nullptr;             // online workspace
     int64_t ws_words = 0;
@@ -270,12 +293,9 @@ static psml_status deal_prg(psml_model_s *m, DealItem &it, uint64_t cid, cudaStr
     return PSML_OK;
 }
 
-static psml_status deal_item(psml_model_s *m, DealItem &it, uint32_t step, cudaStream_t s) {
-    const uint64_t seed = m->d.dealer_seed;
-    const uint64_t cid = call_id(m->d.pair_id, step, it.layer, it.op, it.slot);
-    switch (it.kind) {
-    case IT_MATRIX: {
-        PSML_TRY(deal_prg(m, it, cid, s));
+// Z = U V part of a matrix / conv triplet (after its PRG part)
+static psml_status deal_gemm(psml_model_s *m, DealItem &it, cudaStream_t s) {
+    if (it.kind == IT_MATRIX) {
         if (m->ctx->use_tc(it.M, it.K, it.N))
             return tc_dealer_gemm(64, it.U.p[0], it.U.p[1], it.V.p[0], it.V.p[1], it.M, it.K, it.N, it.Z.p[0],
                                   it.Z.p[1], m->dws, sizeof(T) * (size_t)m->dws_words, s);
@@ -285,15 +305,22 @@ static psml_status deal_item(psml_model_s *m, DealItem &it, uint32_t step, cudaS
         ops.M = it.M; ops.N = it.N; ops.Kext = it.K;
         return launch_ring_gemm<T, DealerOps<T>>(ops, m->dws, m->dws_words, s, m->ctx->sm_count);
     }
+    ConvDealerOps<T> ops;   // Z_1 = im2col(U_0 + U_1) (^T) (V_0 + V_1) - Z_0
+    ops.U0 = it.U.p[0]; ops.U1 = it.U.p[1]; ops.V0 = it.V.p[0]; ops.V1 = it.V.p[1];
+    ops.Z0 = it.Z.p[0]; ops.Z1 = it.Z.p[1];
+    ops.g = m->g; ops.M = it.M; ops.N = it.N; ops.Kext = it.K; ops.transposed = it.kind == IT_CONV_GW;
+    return launch_ring_gemm<T, ConvDealerOps<T>>(ops, m->dws, m->dws_words, s, m->ctx->sm_count);
+}
+
+static psml_status deal_item(psml_model_s *m, DealItem &it, uint32_t step, cudaStream_t s) {
+    const uint64_t seed = m->d.dealer_seed;
+    const uint64_t cid = call_id(m->d.pair_id, step, it.layer, it.op, it.slot);
+    switch (it.kind) {
+    case IT_MATRIX:
     case IT_CONV_FWD:
-    case IT_CONV_GW: {
+    case IT_CONV_GW:
         PSML_TRY(deal_prg(m, it, cid, s));
-        ConvDealerOps<T> ops;   // Z_1 = im2col(U_0 + U_1) (^T) (V_0 + V_1) - Z_0
-        ops.U0 = it.U.p[0]; ops.U1 = it.U.p[1]; ops.V0 = it.V.p[0]; ops.V1 = it.V.p[1];
-        ops.Z0 = it.Z.p[0]; ops.Z1 = it.Z.p[1];
-        ops.g = m->g; ops.M = it.M; ops.N = it.N; ops.Kext = it.K; ops.transposed = it.kind == IT_CONV_GW;
-        return launch_ring_gemm<T, ConvDealerOps<T>>(ops, m->dws, m->dws_words, s, m->ctx->sm_count);
-    }
+        return deal_gemm(m, it, s);
     case IT_HAD: {
         ProfScope prof(PROF_DEALER, s, (double)sizeof(T) * 6 * it.n);
         void *U[2] = {it.U.p[0], it.U.p[1]}, *V[2] = {it.V.p[0], it.V.p[1]}, *Z[2] = {it.Z.p[0], it.Z.p[1]};
@@ -308,11 +335,108 @@ static psml_status deal_item(psml_model_s *m, DealItem &it, uint32_t step, cudaS
     return PSML_OK;
 }
 
-static psml_status deal_pool(psml_model_s *m, int pool, uint32_t step, bool infer_only, cudaStream_t s) {
-    for (auto &it : m->items[pool]) {
+// Work lists of the fused dealer for items[pool] (step field of the call ids filled in on device).
+static psml_status build_plan(psml_model_s *m, int pool, bool infer_only) {
+    DealPlan &P = m->plan[pool][infer_only ? 1 : 0];
+    std::vector<PrgJob> pj;
+    std::vector<GemmJob> gj;
+    auto job = [&](int kind, std::initializer_list<uint32_t> tags, uint64_t cid, int64_t n,
+                   std::initializer_list<T *> outs) {
+        if (n <= 0) return;
+        PrgJob j{};
+        j.kind = kind;
+        int i = 0;
+        for (uint32_t t : tags) j.tag[i++] = t;
+        i = 0;
+        for (T *o : outs) j.out[i++] = o;
+        j.cid = cid; j.n = n; j.blk_begin = P.prg_blocks;
+        P.prg_blocks += (n + 7) / 8;
+        pj.push_back(j);
+    };
+    const int L = 6;   // log2(64): 2L AND triplets + one daBit per element (R9)
+    auto &items = m->items[pool];
+    for (size_t k = 0; k < items.size(); ++k) {
+        DealItem &it = items[k];
         if (infer_only && !it.fwd) continue;
-        PSML_TRY(deal_item(m, it, step, s));
+        const uint64_t cid = call_id(m->d.pair_id, 0, it.layer, it.op, it.slot);
+        switch (it.kind) {
+        case IT_MATRIX:
+        case IT_CONV_FWD:
+        case IT_CONV_GW:
+            job(PJ_PAIR, {TAG_U0, TAG_U1}, cid, it.U.n, {it.U.p[0], it.U.p[1]});
+            job(PJ_PAIR, {TAG_V0, TAG_V1}, cid, it.V.n, {it.V.p[0], it.V.p[1]});
+            job(PJ_SINGLE, {TAG_Z0}, cid, it.Z.n, {it.Z.p[0]});
+            if (it.kind == IT_MATRIX && !m->ctx->use_tc(it.M, it.K, it.N) && it.M * it.N > 0) {
+                GemmJob g{};
+                g.U0 = it.U.p[0]; g.U1 = it.U.p[1]; g.V0 = it.V.p[0]; g.V1 = it.V.p[1];
+                g.Z0 = it.Z.p[0]; g.Z1 = it.Z.p[1];
+                g.M = it.M; g.K = it.K; g.N = it.N;
+                g.tiles_n = (int)((it.N + 15) / 16);
+                g.tile_begin = P.gemm_tiles;
+                P.gemm_tiles += ((it.M + 15) / 16) * g.tiles_n;
+                gj.push_back(g);
+            } else {
+                P.rest.push_back((int)k);
+            }
+            break;
+        case IT_HAD:
+            job(PJ_HAD, {TAG_U0, TAG_U1, TAG_V0, TAG_V1, TAG_Z0}, cid, it.n,
+                {it.U.p[0], it.U.p[1], it.V.p[0], it.V.p[1], it.Z.p[0], it.Z.p[1]});
+            break;
+        case IT_MSB: {
+            T *m0 = it.mat.p[0], *m1 = it.mat.p[1];
+            const int64_t n = it.n;
+            for (int t = 0; t < 2 * L; ++t) {
+                const int64_t o = (int64_t)t * 3 * n;
+                job(PJ_AND, {tag4('a', '0', t), tag4('a', '1', t), tag4('b', '0', t), tag4('b', '1', t), tag4('c', '0', t)},
+                    cid, n, {m0 + o, m1 + o, m0 + o + n, m1 + o + n, m0 + o + 2 * n, m1 + o + 2 * n});
+            }
+            const int64_t o = (int64_t)2 * L * 3 * n;
+            job(PJ_DABIT, {TAG_R0, TAG_R1, TAG_RA}, cid, n, {m0 + o, m1 + o, m0 + o + n, m1 + o + n});
+            break;
+        }
+        }
     }
+    P.n_prg = (int)pj.size();
+    P.n_gemm = (int)gj.size();
+    if (P.n_prg) {
+        T *d = nullptr;
+        PSML_TRY(dalloc(m, &d, (int64_t)((sizeof(PrgJob) * pj.size() + 7) / 8)));
+        PSML_CUDA_TRY(cudaMemcpy(d, pj.data(), sizeof(PrgJob) * pj.size(), cudaMemcpyHostToDevice));
+        P.prg = (PrgJob *)d;
+    }
+    if (P.n_gemm) {
+        T *d = nullptr;
+        PSML_TRY(dalloc(m, &d, (int64_t)((sizeof(GemmJob) * gj.size() + 7) / 8)));
+        PSML_CUDA_TRY(cudaMemcpy(d, gj.data(), sizeof(GemmJob) * gj.size(), cudaMemcpyHostToDevice));
+        P.gemm = (GemmJob *)d;
+    }
+    return PSML_OK;
+}
+
+static psml_status deal_pool(psml_model_s *m, int pool, uint32_t step, bool infer_only, cudaStream_t s) {
+    if (!fused_deal()) {
+        for (auto &it : m->items[pool]) {
+            if (infer_only && !it.fwd) continue;
+            PSML_TRY(deal_item(m, it, step, s));
+        }
+        return PSML_OK;
+    }
+    (void)step;   // the step field comes from m->step_dev (set by the caller / the graph)
+    DealPlan &P = m->plan[pool][infer_only ? 1 : 0];
+    {
+        ProfScope prof(PROF_DEALER, s, 0.0);
+        if (P.n_prg) {
+            deal_prg_kernel<<<(unsigned)((P.prg_blocks + 127) / 128), 128, 0, s>>>(P.prg, P.n_prg, P.prg_blocks,
+                                                                                m->d.dealer_seed, m->step_dev);
+            PSML_LAUNCH_CHECK();
+        }
+        if (P.n_gemm) {
+            deal_gemm_kernel<<<(unsigned)P.gemm_tiles, 256, 0, s>>>(P.gemm, P.n_gemm);
+            PSML_LAUNCH_CHECK();
+        }
+    }
+    for (int k : P.rest) PSML_TRY(deal_gemm(m, m->items[pool][k], s));
     return PSML_OK;
 }
 
@@ -531,6 +655,8 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
     m->items[1] = m->items[0];
     PSML_TRY(alloc_items(mp, m->items[0]));
     PSML_TRY(alloc_items(mp, m->items[1]));
+    for (int pl = 0; pl < 2; ++pl)
+        for (int inf = 0; inf < 2; ++inf) PSML_TRY(build_plan(mp, pl, inf != 0));
     m->dws_words = dws_need(mp);
     PSML_TRY(dalloc(mp, &m->dws, m->dws_words));
     PSML_CUDA_TRY(cudaStreamCreateWithFlags(&m->side, cudaStreamNonBlocking));

@@ -1,0 +1,12 @@
+cd $GRAFT_REPO_ROOT
+timeout 600 python -m pytest tests/test_gpu_training.py -q -x -k "graph or bitexact or explicit" 2>&1 | tail -5
+timeout 300 python bench.py --steps 2000 --no-cpu-baseline --no-ring-gemm > gpurun_out/b33.json 2> gpurun_out/b33.err
+tail -2 gpurun_out/b33.err
+python -c "
+import json; d=json.load(open('gpurun_out/b33.json'))
+print('value',d['value'],'online_graph',d.get('online_graph_samples_per_s'),'online',d['online_samples_per_s'],'e2e',d['e2e']['value'],'ms',d['ms_per_step'],'nodes',d['gpu_launches'])
+for k,v in d['kernel_classes'].items(): print(k, round(v['ms_per_step'],4), round(v['ms_per_launch'],4), v['launches_per_step'])"
+PSML_DEAL=items timeout 300 python bench.py --steps 2000 --no-cpu-baseline --no-ring-gemm > gpurun_out/b33i.json 2>/dev/null
+python -c "
+import json; d=json.load(open('gpurun_out/b33i.json'))
+print('ITEMS value',d['value'],'online_graph',d.get('online_graph_samples_per_s'),'ms',d['ms_per_step'],'nodes',d['gpu_launches'])"
