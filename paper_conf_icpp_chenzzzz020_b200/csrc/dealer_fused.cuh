@@ -2,8 +2,8 @@
 //   deal_prg_kernel   one work list over every PRG stream of the step (matrix U/V pairs, Z_0,
 //                     Hadamard triplets with Z_1, boolean AND triplets with c_1, daBits); each
 //                     thread produces one ChaCha20 block's worth of every stream of its job
-//   deal_gemm_kernel  grouped Z_1 = (U_0 + U_1)(V_0 + V_1) - Z_0 over all matrix triplets, one
-//                     16 x 16 output tile per CTA, job found from the tile index
+//   ring_gemm_cl_grouped<DealerOps> (gemm_cl.cuh) then computes Z_1 = (U_0 + U_1)(V_0 + V_1) - Z_0
+//                     for every matrix triplet of the step in one cluster-split-K launch
 // Same streams, call ids and arithmetic as the per-item dealer (bit-identical, tested); the step
 // field of every call id comes from the model's device word (one captured graph serves all steps).
 #pragma once
@@ -20,14 +20,6 @@ struct PrgJob {
     int64_t n;            // elements
     int64_t blk_begin;    // first global block of this job
     uint64_t *out[6];
-};
-
-struct GemmJob {
-    const uint64_t *U0, *U1, *V0, *V1, *Z0;
-    uint64_t *Z1;
-    int64_t M, K, N;
-    int64_t tile_begin;   // first global 16 x 16 tile of this job
-    int tiles_n;
 };
 
 __device__ __forceinline__ uint64_t cid_with_step(uint64_t cid, const uint32_t *step) {
@@ -76,40 +68,6 @@ __global__ void __launch_bounds__(128) deal_prg_kernel(const PrgJob *__restrict_
             }
         }
     }
-}
-
-__global__ void __launch_bounds__(256) deal_gemm_kernel(const GemmJob *__restrict__ jobs, int njobs) {
-    __shared__ uint64_t As[16][65];
-    __shared__ uint64_t Bs[64][16];
-    const int64_t t = blockIdx.x;
-    int lo = 0, hi = njobs - 1;
-    while (lo < hi) {
-        const int mid = (lo + hi + 1) >> 1;
-        if (jobs[mid].tile_begin <= t) lo = mid; else hi = mid - 1;
-    }
-    const GemmJob J = jobs[lo];
-    const int64_t tt = t - J.tile_begin;
-    const int64_t m0 = (tt / J.tiles_n) * 16, n0 = (tt % J.tiles_n) * 16;
-    const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
-    uint64_t acc = 0;
-    for (int64_t k0 = 0; k0 < J.K; k0 += 64) {
-#pragma unroll
-        for (int r = 0; r < 4; ++r) {
-            const int idx = tid + r * 256;
-            const int mm = idx >> 6, kk = idx & 63;
-            const int64_t m = m0 + mm, k = k0 + kk;
-            As[mm][kk] = (m < J.M && k < J.K) ? J.U0[m * J.K + k] + J.U1[m * J.K + k] : 0;
-            const int kb = idx >> 4, nn = idx & 15;
-            const int64_t k2 = k0 + kb, n = n0 + nn;
-            Bs[kb][nn] = (n < J.N && k2 < J.K) ? J.V0[k2 * J.N + n] + J.V1[k2 * J.N + n] : 0;
-        }
-        __syncthreads();
-#pragma unroll 16
-        for (int kk = 0; kk < 64; ++kk) acc += As[ty][kk] * Bs[kk][tx];
-        __syncthreads();
-    }
-    const int64_t m = m0 + ty, n = n0 + tx;
-    if (m < J.M && n < J.N) J.Z1[m * J.N + n] = acc - J.Z0[m * J.N + n];
 }
 
 }  // namespace psml

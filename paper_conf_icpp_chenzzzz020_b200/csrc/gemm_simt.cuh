@@ -12,6 +12,7 @@
 // exact), finished by ring_gemm_finalize which applies the epilogue.
 #pragma once
 #include <algorithm>
+#include <cstdlib>
 
 #include "common.cuh"
 
@@ -29,6 +30,8 @@ struct PlainOps {
     static constexpr int nparty = 1;
     __device__ __forceinline__ T a(int, int64_t m, int64_t k) const { return A[m * Kext + k]; }
     __device__ __forceinline__ T b(int, int64_t k, int64_t n) const { return B[k * N + n]; }
+    __device__ __forceinline__ T zload(int, int64_t, int64_t) const { return 0; }
+    __device__ __forceinline__ void put(int, int64_t m, int64_t n, T acc, T) const { C[m * N + n] = acc; }
     __device__ __forceinline__ void store(int, int64_t m, int64_t n, T acc) const { C[m * N + n] = acc; }
 };
 
@@ -47,6 +50,8 @@ struct DealerOps {
     __device__ __forceinline__ T b(int, int64_t k, int64_t n) const {
         return V0[k * N + n] + V1[k * N + n];
     }
+    __device__ __forceinline__ T zload(int, int64_t m, int64_t n) const { return Z0[m * N + n]; }
+    __device__ __forceinline__ void put(int, int64_t m, int64_t n, T acc, T z) const { Z1[m * N + n] = acc - z; }
     __device__ __forceinline__ void store(int, int64_t m, int64_t n, T acc) const {
         Z1[m * N + n] = acc - Z0[m * N + n];
     }
@@ -55,33 +60,35 @@ struct DealerOps {
 // Beaver product, both parties, Eq. 8 shape.  E/F are opened on the fly from the two parties'
 // messages mE[0], mE[1] (M x K) and mF[0], mF[1] (K x N).  form 0 (BJ canonical):
 //   [i.E + U_i | E] . [F ; V_i];  form 1 (Eq. 6/8): [A_i - i.E | E] . [F ; B_i].
-template <typename T>
+template <typename T, int FORM = 0>
 struct BeaverOps {
     const T *mE0, *mE1, *mF0, *mF1;
     const T *U[2], *V[2], *Z[2];
     const T *A[2], *B[2];   // only for form 1 (op(A) / op(B) layouts, see transA/transB)
     T *C[2];
     int64_t M, N, K, Kext;  // Kext = 2K
-    int form, transA, transB, trunc;
+    int transA, transB, trunc;
+    static constexpr int form = FORM;   // compile time: no branch in the loaders
     static constexpr int nparty = 2;
-    __device__ __forceinline__ T opA(int p, int64_t m, int64_t k) const {
-        return transA ? A[p][k * M + m] : A[p][m * K + k];
-    }
-    __device__ __forceinline__ T opB(int p, int64_t k, int64_t n) const {
-        return transB ? B[p][n * K + k] : B[p][k * N + n];
-    }
+    // Branch-free loaders (every load issued unconditionally at a valid address, the result
+    // selected afterwards) so a thread's operand loads overlap instead of serialising.
     __device__ __forceinline__ T a(int p, int64_t m, int64_t k) const {
-        if (k < K) {
-            T e = mE0[m * K + k] + mE1[m * K + k];
-            return form == 0 ? (T)((T)p * e + U[p][m * K + k]) : (T)(opA(p, m, k) - (T)p * e);
-        }
-        k -= K;
-        return mE0[m * K + k] + mE1[m * K + k];
+        const bool first = k < K;
+        const int64_t kk = first ? k : k - K, i = m * K + kk;
+        const T e = mE0[i] + mE1[i];
+        const T x = form == 0 ? U[p][i] : A[p][transA ? kk * M + m : i];
+        return first ? (form == 0 ? (T)((T)p * e + x) : (T)(x - (T)p * e)) : e;
     }
     __device__ __forceinline__ T b(int p, int64_t k, int64_t n) const {
-        if (k < K) return mF0[k * N + n] + mF1[k * N + n];
-        k -= K;
-        return form == 0 ? V[p][k * N + n] : opB(p, k, n);
+        const bool first = k < K;
+        const int64_t kk = first ? k : k - K, i = kk * N + n;
+        const T *second = form == 0 ? V[p] + i : B[p] + (transB ? n * K + kk : i);
+        const T x = *(first ? mF0 + i : second), y = mF1[i];
+        return first ? (T)(x + y) : x;
+    }
+    __device__ __forceinline__ T zload(int p, int64_t m, int64_t n) const { return Z[p][m * N + n]; }
+    __device__ __forceinline__ void put(int p, int64_t m, int64_t n, T acc, T z) const {
+        C[p][m * N + n] = trunc_share<T>(acc + z, p, trunc);
     }
     __device__ __forceinline__ void store(int p, int64_t m, int64_t n, T acc) const {
         T c = acc + Z[p][m * N + n];
@@ -111,14 +118,21 @@ struct BeaverFusedOps {
     }
     __device__ __forceinline__ T a(int p, int64_t m, int64_t k) const {
         const bool first = k < K;
-        if (!first) k -= K;
-        const int64_t u = m * K + k;
-        const T e = (opA(0, m, k) - U[0][u]) + (opA(1, m, k) - U[1][u]);
-        return first ? (T)((T)p * e + U[p][u]) : e;
+        const int64_t kk = first ? k : k - K, u = m * K + kk;
+        const T u0 = U[0][u], u1 = U[1][u];
+        const T e = (opA(0, m, kk) - u0) + (opA(1, m, kk) - u1);
+        return first ? (T)((T)p * e + (p ? u1 : u0)) : e;
     }
     __device__ __forceinline__ T b(int p, int64_t k, int64_t n) const {
-        if (k < K) return (opB(0, k, n) - V[0][k * N + n]) + (opB(1, k, n) - V[1][k * N + n]);
-        return V[p][(k - K) * N + n];
+        const bool first = k < K;
+        const int64_t kk = first ? k : k - K, i = kk * N + n;
+        const T v0 = V[0][i], v1 = V[1][i];
+        const T f = (opB(0, kk, n) - v0) + (opB(1, kk, n) - v1);
+        return first ? f : (p ? v1 : v0);
+    }
+    __device__ __forceinline__ T zload(int p, int64_t m, int64_t n) const { return Z[p][m * N + n]; }
+    __device__ __forceinline__ void put(int p, int64_t m, int64_t n, T acc, T z) const {
+        C[p][m * N + n] = trunc_share<T>(acc + z, p, trunc);
     }
     __device__ __forceinline__ void store(int p, int64_t m, int64_t n, T acc) const {
         C[p][m * N + n] = trunc_share<T>(acc + Z[p][m * N + n], p, trunc);
@@ -141,16 +155,20 @@ struct BeaverOps1 {
     int party, trunc;
     static constexpr int nparty = 1;
     __device__ __forceinline__ T a(int, int64_t m, int64_t k) const {
-        if (k < K) {
-            const T e = mE0[m * K + k] + mE1[m * K + k];
-            return (T)((T)party * e + U[m * K + k]);
-        }
-        k -= K;
-        return mE0[m * K + k] + mE1[m * K + k];
+        const bool first = k < K;
+        const int64_t kk = first ? k : k - K, i = m * K + kk;
+        const T e = mE0[i] + mE1[i], u = U[i];
+        return first ? (T)((T)party * e + u) : e;
     }
     __device__ __forceinline__ T b(int, int64_t k, int64_t n) const {
-        if (k < K) return mF0[k * N + n] + mF1[k * N + n];
-        return V[(k - K) * N + n];
+        const bool first = k < K;
+        const int64_t kk = first ? k : k - K, i = kk * N + n;
+        const T x = *(first ? mF0 + i : V + i), y = mF1[i];
+        return first ? (T)(x + y) : x;
+    }
+    __device__ __forceinline__ T zload(int, int64_t m, int64_t n) const { return Z[m * N + n]; }
+    __device__ __forceinline__ void put(int, int64_t m, int64_t n, T acc, T z) const {
+        C[m * N + n] = trunc_share<T>(acc + z, party, trunc);
     }
     __device__ __forceinline__ void store(int, int64_t m, int64_t n, T acc) const {
         C[m * N + n] = trunc_share<T>(acc + Z[m * N + n], party, trunc);
@@ -188,16 +206,21 @@ struct ConvBeaverOps {
     static constexpr int nparty = 2;
     __device__ __forceinline__ int64_t src(int64_t r, int64_t c) const { return conv_src(g, r, c); }
     __device__ __forceinline__ T a(int p, int64_t m, int64_t k) const {
-        bool first = k < K;
-        if (!first) k -= K;
-        int64_t s = transposed ? src(k, m) : src(m, k);
-        T e = mE0[s] + mE1[s];
-        return first ? (T)((T)p * e + UX[p][s]) : e;
+        const bool first = k < K;
+        const int64_t kk = first ? k : k - K;
+        const int64_t s = transposed ? src(kk, m) : src(m, kk);
+        const T e = mE0[s] + mE1[s], u = UX[p][s];
+        return first ? (T)((T)p * e + u) : e;
     }
     __device__ __forceinline__ T b(int p, int64_t k, int64_t n) const {
-        if (k < K) return mF0[k * N + n] + mF1[k * N + n];
-        k -= K;
-        return V[p][k * N + n];
+        const bool first = k < K;
+        const int64_t kk = first ? k : k - K, i = kk * N + n;
+        const T x = *(first ? mF0 + i : V[p] + i), y = mF1[i];
+        return first ? (T)(x + y) : x;
+    }
+    __device__ __forceinline__ T zload(int p, int64_t m, int64_t n) const { return Z[p][m * N + n]; }
+    __device__ __forceinline__ void put(int p, int64_t m, int64_t n, T acc, T z) const {
+        C[p][m * N + n] = trunc_share<T>(acc + z, p, trunc);
     }
     __device__ __forceinline__ void store(int p, int64_t m, int64_t n, T acc) const {
         T c = acc + Z[p][m * N + n];
@@ -223,6 +246,8 @@ struct ConvDealerOps {
     __device__ __forceinline__ T b(int, int64_t k, int64_t n) const {
         return V0[k * N + n] + V1[k * N + n];
     }
+    __device__ __forceinline__ T zload(int, int64_t m, int64_t n) const { return Z0[m * N + n]; }
+    __device__ __forceinline__ void put(int, int64_t m, int64_t n, T acc, T z) const { Z1[m * N + n] = acc - z; }
     __device__ __forceinline__ void store(int, int64_t m, int64_t n, T acc) const {
         Z1[m * N + n] = acc - Z0[m * N + n];
     }
@@ -262,14 +287,16 @@ ring_gemm_tiled(Ops ops, int64_t k_per_split, T *__restrict__ partial) {
             int idx = tid + t * NT;
             int mm = idx / BK, kk = idx % BK;          // coalesced along k
             int64_t m = m0 + mm, k = k0 + kk;
-            ra[t] = (m < ops.M && k < kend) ? ops.a(p, m, k) : (T)0;
+            const T v = ops.a(p, m < ops.M ? m : ops.M - 1, k < kend ? k : kend - 1);
+            ra[t] = (m < ops.M && k < kend) ? v : (T)0;
         }
 #pragma unroll
         for (int t = 0; t < B_PER; ++t) {
             int idx = tid + t * NT;
             int kk = idx / BN, nn = idx % BN;          // coalesced along n
             int64_t k = k0 + kk, n = n0 + nn;
-            rb[t] = (n < ops.N && k < kend) ? ops.b(p, k, n) : (T)0;
+            const T v = ops.b(p, k < kend ? k : kend - 1, n < ops.N ? n : ops.N - 1);
+            rb[t] = (n < ops.N && k < kend) ? v : (T)0;
         }
     };
     auto stash = [&](int buf) {
@@ -313,6 +340,15 @@ ring_gemm_tiled(Ops ops, int64_t k_per_split, T *__restrict__ partial) {
         }
     }
     if (partial == nullptr) {
+        // epilogue operands first (clamped, unconditional), then the stores: no serialised loads
+        T z[TM][TN];
+#pragma unroll
+        for (int i = 0; i < TM; ++i)
+#pragma unroll
+            for (int j = 0; j < TN; ++j) {
+                const int64_t m = m0 + ty + i * (BM / TM), n = n0 + tx + j * (BN / TN);
+                z[i][j] = ops.zload(p, m < ops.M ? m : ops.M - 1, n < ops.N ? n : ops.N - 1);
+            }
 #pragma unroll
         for (int i = 0; i < TM; ++i) {
             int64_t m = m0 + ty + i * (BM / TM);
@@ -320,7 +356,7 @@ ring_gemm_tiled(Ops ops, int64_t k_per_split, T *__restrict__ partial) {
 #pragma unroll
             for (int j = 0; j < TN; ++j) {
                 int64_t n = n0 + tx + j * (BN / TN);
-                if (n < ops.N) ops.store(p, m, n, acc[i][j]);
+                if (n < ops.N) ops.put(p, m, n, acc[i][j], z[i][j]);
             }
         }
     } else {
@@ -375,10 +411,12 @@ __global__ void __launch_bounds__(256) ring_gemm_small(Ops ops, int64_t k_per_sp
             int mm, kk, kb, nn;
             amap(idx, mm, kk);
             const int64_t m = m0 + mm, k = k0 + kk;
-            ra[t] = (m < ops.M && k < kend) ? ops.a(p, m, k) : (T)0;
+            const T va = ops.a(p, m < ops.M ? m : ops.M - 1, k < kend ? k : kend - 1);
+            ra[t] = (m < ops.M && k < kend) ? va : (T)0;
             bmap(idx, kb, nn);
             const int64_t k2 = k0 + kb, n = n0 + nn;
-            rb[t] = (n < ops.N && k2 < kend) ? ops.b(p, k2, n) : (T)0;
+            const T vb = ops.b(p, k2 < kend ? k2 : kend - 1, n < ops.N ? n : ops.N - 1);
+            rb[t] = (n < ops.N && k2 < kend) ? vb : (T)0;
         }
     };
     auto stash = [&](int buf) {
@@ -475,6 +513,21 @@ __global__ void ring_gemm_finalize(Ops ops, const T *__restrict__ partial) {
     }
 }
 
+}  // namespace psml
+#include "gemm_cl.cuh"
+namespace psml {
+
+// PSML_SIMT=small: route small products to the 16 x 16 one-output-per-thread kernel instead of
+// the cluster split-K kernel (A/B switch; both bit-identical).
+inline bool simt_cl_enabled() {
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("PSML_SIMT");
+        v = (e && e[0] == 's') ? 0 : 1;
+    }
+    return v == 1;
+}
+
 // ---------------------------------------------------------------------------------------------
 // host-side dispatcher: picks kernel, tile and split-K; `ws` must hold nparty*M*N words when
 // split-K is chosen (ws_words reports the need; pass ws = nullptr to query).
@@ -492,6 +545,10 @@ psml_status launch_ring_gemm(const Ops &ops, T *ws, int64_t ws_words, cudaStream
     // the 16 x 16 small-tile kernel for small outputs or skinny outputs with many rows (CNN conv
     // im2col GEMMs), the 64 x 64 register-blocked kernel otherwise.
     const bool gemv = N <= 2 && M * Ops::nparty <= 4096 && Kx <= 8192;
+    if (!gemv && M * N * Ops::nparty <= ((int64_t)1 << 19) && simt_cl_enabled()) {
+        ProfScope prof(PROF_GEMM, stream, (double)M * N * Kx * Ops::nparty);
+        return launch_ring_gemm_cl<T, Ops>(ops, stream, sm_count);
+    }
     const bool small = !gemv && (N <= 16 || M * N * Ops::nparty <= ((int64_t)1 << 18));
     int splits = 1;
     if (small) {

@@ -75,8 +75,8 @@ struct DealPlan {   // fused dealer of one pool (full or inference-only)
     PrgJob *prg = nullptr;
     int n_prg = 0;
     int64_t prg_blocks = 0;
-    GemmJob *gemm = nullptr;
-    int n_gemm = 0;
+    ClJob<DealerOps<T>> *gemm = nullptr;
+    int n_gemm = 0, gemm_ks = 4;
     int64_t gemm_tiles = 0;
     std::vector<int> rest;   // items whose Z = U V runs in its own launch (conv, tcgen05-sized)
 };
@@ -339,7 +339,7 @@ static psml_status deal_item(psml_model_s *m, DealItem &it, uint32_t step, cudaS
 static psml_status build_plan(psml_model_s *m, int pool, bool infer_only) {
     DealPlan &P = m->plan[pool][infer_only ? 1 : 0];
     std::vector<PrgJob> pj;
-    std::vector<GemmJob> gj;
+    std::vector<ClJob<DealerOps<T>>> gj;
     auto job = [&](int kind, std::initializer_list<uint32_t> tags, uint64_t cid, int64_t n,
                    std::initializer_list<T *> outs) {
         if (n <= 0) return;
@@ -367,13 +367,14 @@ static psml_status build_plan(psml_model_s *m, int pool, bool infer_only) {
             job(PJ_PAIR, {TAG_V0, TAG_V1}, cid, it.V.n, {it.V.p[0], it.V.p[1]});
             job(PJ_SINGLE, {TAG_Z0}, cid, it.Z.n, {it.Z.p[0]});
             if (it.kind == IT_MATRIX && !m->ctx->use_tc(it.M, it.K, it.N) && it.M * it.N > 0) {
-                GemmJob g{};
-                g.U0 = it.U.p[0]; g.U1 = it.U.p[1]; g.V0 = it.V.p[0]; g.V1 = it.V.p[1];
-                g.Z0 = it.Z.p[0]; g.Z1 = it.Z.p[1];
-                g.M = it.M; g.K = it.K; g.N = it.N;
-                g.tiles_n = (int)((it.N + 15) / 16);
+                ClJob<DealerOps<T>> g{};
+                g.ops.U0 = it.U.p[0]; g.ops.U1 = it.U.p[1]; g.ops.V0 = it.V.p[0]; g.ops.V1 = it.V.p[1];
+                g.ops.Z0 = it.Z.p[0]; g.ops.Z1 = it.Z.p[1];
+                g.ops.M = it.M; g.ops.N = it.N; g.ops.Kext = it.K;
+                g.tiles_n = (int)((it.N + ClDefault::BN - 1) / ClDefault::BN);
                 g.tile_begin = P.gemm_tiles;
-                P.gemm_tiles += ((it.M + 15) / 16) * g.tiles_n;
+                g.k_per_split = ((it.K + P.gemm_ks - 1) / P.gemm_ks + ClDefault::BK - 1) / ClDefault::BK * ClDefault::BK;
+                P.gemm_tiles += ((it.M + ClDefault::BM - 1) / ClDefault::BM) * g.tiles_n;
                 gj.push_back(g);
             } else {
                 P.rest.push_back((int)k);
@@ -407,9 +408,10 @@ static psml_status build_plan(psml_model_s *m, int pool, bool infer_only) {
     }
     if (P.n_gemm) {
         T *d = nullptr;
-        PSML_TRY(dalloc(m, &d, (int64_t)((sizeof(GemmJob) * gj.size() + 7) / 8)));
-        PSML_CUDA_TRY(cudaMemcpy(d, gj.data(), sizeof(GemmJob) * gj.size(), cudaMemcpyHostToDevice));
-        P.gemm = (GemmJob *)d;
+        const size_t bytes = sizeof(ClJob<DealerOps<T>>) * gj.size();
+        PSML_TRY(dalloc(m, &d, (int64_t)((bytes + 7) / 8)));
+        PSML_CUDA_TRY(cudaMemcpy(d, gj.data(), bytes, cudaMemcpyHostToDevice));
+        P.gemm = (ClJob<DealerOps<T>> *)d;
     }
     return PSML_OK;
 }
@@ -432,8 +434,17 @@ static psml_status deal_pool(psml_model_s *m, int pool, uint32_t step, bool infe
             PSML_LAUNCH_CHECK();
         }
         if (P.n_gemm) {
-            deal_gemm_kernel<<<(unsigned)P.gemm_tiles, 256, 0, s>>>(P.gemm, P.n_gemm);
-            PSML_LAUNCH_CHECK();
+            cudaLaunchConfig_t cfg = {};
+            cfg.gridDim = dim3((unsigned)P.gemm_tiles, 1, (unsigned)P.gemm_ks);
+            cfg.blockDim = dim3(ClDefault::NT);
+            cfg.stream = s;
+            cudaLaunchAttribute attr[1];
+            attr[0].id = cudaLaunchAttributeClusterDimension;
+            attr[0].val.clusterDim.x = 1; attr[0].val.clusterDim.y = 1; attr[0].val.clusterDim.z = (unsigned)P.gemm_ks;
+            cfg.attrs = attr;
+            cfg.numAttrs = 1;
+            PSML_CUDA_TRY(cudaLaunchKernelEx(&cfg, ring_gemm_cl_grouped<T, DealerOps<T>>, (const ClJob<DealerOps<T>> *)P.gemm,
+                                             P.n_gemm, P.gemm_ks));
         }
     }
     for (int k : P.rest) PSML_TRY(deal_gemm(m, m->items[pool][k], s));

@@ -64,15 +64,18 @@ psml_status beaver_matmul(const T *const A[2], const T *const B[2], const T *con
         mask_kernel<T><<<dim3((unsigned)std::min<int64_t>(maxt, 148 * 8), 1, 4), dim3(32, 8), 0, s>>>(jobs);
         PSML_LAUNCH_CHECK();
     }
-    BeaverOps<T> ops;
-    ops.mE0 = mE0; ops.mE1 = mE1; ops.mF0 = mF0; ops.mF1 = mF1;
-    for (int p = 0; p < 2; ++p) {
-        ops.U[p] = U[p]; ops.V[p] = V[p]; ops.Z[p] = Z[p]; ops.A[p] = A[p]; ops.B[p] = B[p]; ops.C[p] = C[p];
-    }
-    ops.M = M; ops.N = N; ops.K = K; ops.Kext = 2 * K;
-    ops.form = (flags & PSML_PAPER_FORM) ? 1 : 0;
-    ops.transA = tA; ops.transB = tB; ops.trunc = trunc;
-    PSML_TRY((launch_ring_gemm<T, BeaverOps<T>>(ops, partial, ws_words - (partial - ws), s, sm_count)));
+    auto run = [&](auto ops) -> psml_status {
+        using Ops = decltype(ops);
+        ops.mE0 = mE0; ops.mE1 = mE1; ops.mF0 = mF0; ops.mF1 = mF1;
+        for (int p = 0; p < 2; ++p) {
+            ops.U[p] = U[p]; ops.V[p] = V[p]; ops.Z[p] = Z[p]; ops.A[p] = A[p]; ops.B[p] = B[p]; ops.C[p] = C[p];
+        }
+        ops.M = M; ops.N = N; ops.K = K; ops.Kext = 2 * K;
+        ops.transA = tA; ops.transB = tB; ops.trunc = trunc;
+        return launch_ring_gemm<T, Ops>(ops, partial, ws_words - (partial - ws), s, sm_count);
+    };
+    if (flags & PSML_PAPER_FORM) PSML_TRY(run(BeaverOps<T, 1>{}));
+    else PSML_TRY(run(BeaverOps<T, 0>{}));
     if (traceE) {
         for (int p = 0; p < 2; ++p)
             if (traceE[p]) PSML_CUDA_TRY(cudaMemcpyAsync(traceE[p], p ? mE1 : mE0, sizeof(T) * M * K, cudaMemcpyDeviceToDevice, s));
