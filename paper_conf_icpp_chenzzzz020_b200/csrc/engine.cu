@@ -385,6 +385,19 @@ static psml_status open_matmul_t(Ctx *c, int party, const void *Es, const void *
         psml_status st = tc_open_matmul_one(c, 8 * (int)sizeof(T), party, Es, Er, Fs, Fr, U, V, Z, M, K, N, trunc, C, s);
         if (st != PSML_ERR_UNSUPPORTED) return st;
     }
+    if (seg_eligible(M, K, N, 1) && simt_cl_enabled()) {   // open once, then the two-segment GEMM
+        PSML_TRY(c->ensure_ws(sizeof(T) * (2 * M * K + K * N)));
+        T *E = (T *)c->ws, *X = E + M * K, *F = X + M * K;
+        OpenJobs<T> oj;
+        oj.j[0] = {{(const T *)Es, (const T *)Er}, {nullptr, nullptr}, E, X, (const T *)U, (T)party, M, K, 0};
+        oj.j[1] = {{(const T *)Fs, (const T *)Fr}, {nullptr, nullptr}, F, nullptr, nullptr, (T)0, K, N, 0};
+        PSML_TRY(launch_open<T>(oj, s));
+        SegArgs<T> sa{};
+        sa.X[0] = X; sa.E = E; sa.F = F; sa.V[0] = (const T *)V; sa.Z[0] = (const T *)Z; sa.C[0] = (T *)C;
+        sa.party[0] = party;
+        sa.M = M; sa.N = N; sa.K = K; sa.trunc = trunc;
+        return launch_seg_gemm<T>(sa, 1, s, c->sm_count);
+    }
     PSML_TRY(c->ensure_ws(sizeof(T) * M * N));
     BeaverOps1<T> ops;
     ops.mE0 = (const T *)Es; ops.mE1 = (const T *)Er; ops.mF0 = (const T *)Fs; ops.mF1 = (const T *)Fr;

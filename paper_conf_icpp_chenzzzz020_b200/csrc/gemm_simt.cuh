@@ -515,6 +515,7 @@ __global__ void ring_gemm_finalize(Ops ops, const T *__restrict__ partial) {
 
 }  // namespace psml
 #include "gemm_cl.cuh"
+#include "gemm_seg.cuh"
 namespace psml {
 
 // PSML_SIMT=small: route small products to the 16 x 16 one-output-per-thread kernel instead of

@@ -49,9 +49,36 @@ psml_status beaver_matmul(const T *const A[2], const T *const B[2], const T *con
                           int64_t N, int flags, int trunc, T *const C[2], T *ws, int64_t ws_words,
                           cudaStream_t s, int sm_count, T *const traceE[2] = nullptr,
                           T *const traceF[2] = nullptr) {
+    const int tA = (flags & PSML_TRANS_A) ? 1 : 0, tB = (flags & PSML_TRANS_B) ? 1 : 0;
+    if (!(flags & PSML_PAPER_FORM) && seg_eligible(M, K, N, 2) && simt_cl_enabled()) {
+        // open once (E, X_1 = E + U_1, F), then C_p = [X_p | E] . [F ; V_p] + Z_p (gemm_seg.cuh)
+        T *E = ws, *X1 = ws + M * K, *F = ws + 2 * M * K;
+        OpenJobs<T> oj;
+        oj.j[0] = {{A[0], A[1]}, {U[0], U[1]}, E, X1, U[1], (T)1, M, K, tA};
+        oj.j[1] = {{B[0], B[1]}, {V[0], V[1]}, F, nullptr, nullptr, (T)0, K, N, tB};
+        PSML_TRY(launch_open<T>(oj, s));
+        const bool tE = traceE && traceE[0] && traceE[1], tF = traceF && traceF[0] && traceF[1];
+        if (tE || tF) {   // the parties' masked messages E_i, F_i for the trace (tests only)
+            MaskJobs<T> tj;
+            tj.j[0] = {A[0], U[0], tE ? traceE[0] : nullptr, M, K, tA};
+            tj.j[1] = {A[1], U[1], tE ? traceE[1] : nullptr, M, K, tA};
+            tj.j[2] = {B[0], V[0], tF ? traceF[0] : nullptr, K, N, tB};
+            tj.j[3] = {B[1], V[1], tF ? traceF[1] : nullptr, K, N, tB};
+            const int first = tE ? 0 : 2, count = (tE ? 2 : 0) + (tF ? 2 : 0);
+            for (int q = 0; q < count; ++q) tj.j[q] = tj.j[first + q];
+            tj.count = count;
+            const int64_t maxt = std::max(((M + 31) / 32) * ((K + 31) / 32), ((K + 31) / 32) * ((N + 31) / 32));
+            mask_kernel<T><<<dim3((unsigned)std::min<int64_t>(maxt, 148 * 8), 1, (unsigned)count), dim3(32, 8), 0, s>>>(tj);
+            PSML_LAUNCH_CHECK();
+        }
+        SegArgs<T> sa;
+        sa.X[0] = U[0]; sa.X[1] = X1; sa.E = E; sa.F = F;
+        for (int p = 0; p < 2; ++p) { sa.V[p] = V[p]; sa.Z[p] = Z[p]; sa.C[p] = C[p]; sa.party[p] = p; }
+        sa.M = M; sa.N = N; sa.K = K; sa.trunc = trunc;
+        return launch_seg_gemm<T>(sa, 2, s, sm_count);
+    }
     T *mE0 = ws, *mE1 = ws + M * K, *mF0 = ws + 2 * M * K, *mF1 = mF0 + K * N;
     T *partial = mF1 + K * N;
-    const int tA = (flags & PSML_TRANS_A) ? 1 : 0, tB = (flags & PSML_TRANS_B) ? 1 : 0;
     MaskJobs<T> jobs;
     jobs.j[0] = {A[0], U[0], mE0, M, K, tA};
     jobs.j[1] = {A[1], U[1], mE1, M, K, tA};
