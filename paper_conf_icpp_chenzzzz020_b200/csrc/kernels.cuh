@@ -499,14 +499,26 @@ __global__ void __launch_bounds__(256) msb_chain_pair_kernel(MsbArgs<T> a, Chain
     }
     const T *mat = p ? a.mat.p[1] : a.mat.p[0];
     T *msg = p ? a.msg.p[1] : a.msg.p[0];
-    auto M = [&](int t, int w) -> T { return mat[((int64_t)t * 3 + w) * n + e]; };
+    // Every load of the chain is data-independent: issue them all up front (one memory round trip
+    // instead of one per protocol round -- the rounds' message stores would otherwise order them).
+    T mt[2 * L][3];
+#pragma unroll
+    for (int t = 0; t < 2 * L; ++t)
+#pragma unroll
+        for (int w = 0; w < 3; ++w) mt[t][w] = mat[((int64_t)t * 3 + w) * n + e];
+    const int64_t off = (int64_t)2 * L * 3 * n;
+    const T rB = mat[off + e], rA = mat[off + n + e];
+    const T *xin = p ? a.x.p[1] : a.x.p[0];
+    const T half = p == 0 ? a.half : (T)0;
+    const T x = a.mode == 0 ? xin[e] : (e < (n >> 1) ? xin[e] + half : xin[e - (n >> 1)] - half);
+    T hu = 0, hv = 0, hz = 0, ysub = 0;
+    if (MODE != 0) { hu = SEL(o.U)[e]; hv = SEL(o.V)[e]; hz = SEL(o.Z)[e]; }
+    if (MODE == 2 && !second && SEL(o.Ysub)) ysub = SEL(o.Ysub)[e];
+    auto M = [&](int t, int w) -> T { return mt[t][w]; };
     auto z_of = [&](T ee, T ff, int t) -> T {
         T r = (ee & M(t, 1)) ^ (M(t, 0) & ff) ^ M(t, 2);
         return p == 1 ? (T)(r ^ (ee & ff)) : r;
     };
-    const T *xin = p ? a.x.p[1] : a.x.p[0];
-    const T half = p == 0 ? a.half : (T)0;
-    const T x = a.mode == 0 ? xin[e] : (e < (n >> 1) ? xin[e] + half : xin[e - (n >> 1)] - half);
     // round 1: AND t = 0 on X = (x0, 0), Y = (0, x1)
     T m0 = (p == 0 ? x : (T)0) ^ M(0, 0), m1 = (p == 1 ? x : (T)0) ^ M(0, 1);
     if (valid) { msg[e] = m0; msg[n + e] = m1; }
@@ -529,22 +541,21 @@ __global__ void __launch_bounds__(256) msb_chain_pair_kernel(MsbArgs<T> a, Chain
     }
     const T bit = ((x >> (l - 1)) & 1) ^ ((G >> (l - 2)) & 1);
     if (valid && SEL(o.msbB)) SEL(o.msbB)[e] = bit;
-    const int64_t off = (int64_t)2 * L * 3 * n;
-    const T cm = bit ^ mat[off + e];          // B2A: c_i = msb_i ^ rB_i
+    const T cm = bit ^ rB;                    // B2A: c_i = msb_i ^ rB_i
     if (valid) msg[e] = cm;
     const T c = cm ^ peer_of(cm);
-    const T mA = (p == 0 ? c : (T)0) + ((T)1 - (T)2 * c) * mat[off + n + e];
+    const T mA = (p == 0 ? c : (T)0) + ((T)1 - (T)2 * c) * rA;
     if (MODE == 0) {
         if (valid) SEL(o.msbA)[e] = mA;
         return;
     }
     const T d = (p == 0 ? (T)1 : (T)0) - mA;  // DReLU share
     if (valid && SEL(o.drelu)) SEL(o.drelu)[e] = d;
-    const T u = SEL(o.U)[e], v = SEL(o.V)[e];
+    const T u = hu, v = hv;
     const T me = x - u, mf = d - v;           // Hadamard round: mask
     if (valid) { SEL(o.mE)[e] = me; SEL(o.mF)[e] = mf; }
     const T E = me + peer_of(me), F = mf + peer_of(mf);
-    const T r = (T)p * E * F + E * v + u * F + SEL(o.Z)[e];
+    const T r = (T)p * E * F + E * v + u * F + hz;
     if (MODE == 1) {
         if (valid) SEL(o.y)[e] = r;
         return;
@@ -553,7 +564,7 @@ __global__ void __launch_bounds__(256) msb_chain_pair_kernel(MsbArgs<T> a, Chain
     if (valid && !second) {
         const T out = r - r2;                 // ReLU(z + 1/2) - ReLU(z - 1/2)
         if (SEL(o.y)) SEL(o.y)[e] = out;
-        if (SEL(o.delta)) SEL(o.delta)[e] = out - SEL(o.Ysub)[e];
+        if (SEL(o.delta)) SEL(o.delta)[e] = out - ysub;
     }
 }
 

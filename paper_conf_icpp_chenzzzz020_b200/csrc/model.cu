@@ -117,6 +117,8 @@ struct psml_model_s {
     int64_t graph_kernels = 0;
     cudaStream_t side = nullptr;       // dealer branch inside the pipelined graph
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+    cudaStream_t hi = nullptr;         // online phase inside the pipelined graph (highest priority)
+    cudaEvent_t ev_hi = nullptr;
 };
 
 namespace psml {
@@ -429,8 +431,16 @@ static psml_status deal_pool(psml_model_s *m, int pool, uint32_t step, bool infe
     {
         ProfScope prof(PROF_DEALER, s, 0.0);
         if (P.n_prg) {
-            deal_prg_kernel<<<(unsigned)((P.prg_blocks + 127) / 128), 128, 0, s>>>(P.prg, P.n_prg, P.prg_blocks,
-                                                                                m->d.dealer_seed, m->step_dev);
+            // a bounded grid (grid-stride): the PRG work runs beside the online phase instead of
+            // occupying every SM's register file ahead of it (PSML_DEAL_CTAS per SM; 0 = full grid)
+            static int per_sm = -1;
+            if (per_sm < 0) {
+                const char *e = getenv("PSML_DEAL_CTAS");
+                per_sm = e ? atoi(e) : 4;   // measured best of {1, 2, 4, full} (tools/gpu44.sh)
+            }
+            const int64_t full = (P.prg_blocks + 127) / 128;
+            const int64_t grid = per_sm > 0 ? std::min<int64_t>(full, (int64_t)per_sm * m->ctx->sm_count) : full;
+            deal_prg_kernel<<<(unsigned)grid, 128, 0, s>>>(P.prg, P.n_prg, P.prg_blocks, m->d.dealer_seed, m->step_dev);
             PSML_LAUNCH_CHECK();
         }
         if (P.n_gemm) {
@@ -670,7 +680,16 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
         for (int inf = 0; inf < 2; ++inf) PSML_TRY(build_plan(mp, pl, inf != 0));
     m->dws_words = dws_need(mp);
     PSML_TRY(dalloc(mp, &m->dws, m->dws_words));
-    PSML_CUDA_TRY(cudaStreamCreateWithFlags(&m->side, cudaStreamNonBlocking));
+    {
+        // dealer branch at the lowest priority, online branch at the highest: inside the pipelined
+        // graph the block scheduler then serves the online kernels first and the dealer's PRG
+        // work fills the SMs they leave idle (PSML_PRIO=0 disables)
+        int lo = 0, hi = 0;
+        PSML_CUDA_TRY(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+        PSML_CUDA_TRY(cudaStreamCreateWithPriority(&m->side, cudaStreamNonBlocking, lo));
+        PSML_CUDA_TRY(cudaStreamCreateWithPriority(&m->hi, cudaStreamNonBlocking, hi));
+        PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_hi, cudaEventDisableTiming));
+    }
     PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_fork, cudaEventDisableTiming));
     PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_join, cudaEventDisableTiming));
     {
@@ -691,6 +710,8 @@ psml_status psml_model_destroy(psml_model model) {
         if (model->graph[g]) cudaGraphExecDestroy(model->graph[g]);
     if (model->side) cudaStreamDestroy(model->side);
     if (model->ev_fork) cudaEventDestroy(model->ev_fork);
+    if (model->hi) cudaStreamDestroy(model->hi);
+    if (model->ev_hi) cudaEventDestroy(model->ev_hi);
     if (model->ev_join) cudaEventDestroy(model->ev_join);
     for (void *p : model->allocs) cudaFree(p);
     delete model;
@@ -799,14 +820,29 @@ psml_status psml_secure_train_step(psml_model m, const void *const X[2], const v
 // One captured step for online pool `pool`.  Non-pipelined: [dealer(pool)] -> online -> [update].
 // Pipelined: online(pool) -> [update] on `s`, concurrently dealer(1 - pool) for the NEXT step on the
 // side stream (fork/join inside the capture), reading the step word = step + 1.
+static bool use_prio() {
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("PSML_PRIO");
+        v = (e && e[0] == '0') ? 0 : 1;
+    }
+    return v == 1;
+}
+
 static psml_status capture_one(psml_model_s *m, int pool, const T *const X[2], const T *const Y[2], int flags,
                                cudaStream_t s, cudaGraphExec_t *out, int64_t *kernels) {
     const bool pipelined = (flags & 4) != 0;
+    const bool prio = pipelined && use_prio();
     PSML_CUDA_TRY(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
     psml_status st = PSML_OK;
+    cudaStream_t on = s;   // stream of the online phase
     if (pipelined) {
         if (cudaEventRecord(m->ev_fork, s) != cudaSuccess || cudaStreamWaitEvent(m->side, m->ev_fork, 0) != cudaSuccess)
             st = fail(PSML_ERR_CUDA, "graph fork failed");
+        if (st == PSML_OK && prio) {
+            if (cudaStreamWaitEvent(m->hi, m->ev_fork, 0) != cudaSuccess) st = fail(PSML_ERR_CUDA, "graph fork failed");
+            on = m->hi;
+        }
         if (st == PSML_OK) st = deal_pool(m, 1 - pool, 0, false, m->side);
         if (st == PSML_OK && cudaEventRecord(m->ev_join, m->side) != cudaSuccess)
             st = fail(PSML_ERR_CUDA, "graph join record failed");
@@ -814,12 +850,15 @@ static psml_status capture_one(psml_model_s *m, int pool, const T *const X[2], c
         st = deal_pool(m, pool, 0, false, s);
     }
     m->pool = pool;
-    if (st == PSML_OK) st = forward(m, X, Y, nullptr, s);
-    if (st == PSML_OK) st = backward(m, s);
+    if (st == PSML_OK) st = forward(m, X, Y, nullptr, on);
+    if (st == PSML_OK) st = backward(m, on);
     if (st == PSML_OK && (flags & 2)) {
         m->grads_ready = true;
-        st = psml_train_apply_update(m, 0, (psml_stream)s);
+        st = psml_train_apply_update(m, 0, (psml_stream)on);
     }
+    if (prio && st == PSML_OK &&
+        (cudaEventRecord(m->ev_hi, m->hi) != cudaSuccess || cudaStreamWaitEvent(s, m->ev_hi, 0) != cudaSuccess))
+        st = fail(PSML_ERR_CUDA, "graph join failed");
     if (pipelined && st == PSML_OK && cudaStreamWaitEvent(s, m->ev_join, 0) != cudaSuccess)
         st = fail(PSML_ERR_CUDA, "graph join failed");
     cudaGraph_t g = nullptr;
@@ -838,7 +877,8 @@ static psml_status capture_one(psml_model_s *m, int pool, const T *const X[2], c
         cudaGraphNodeType t;
         if (cudaGraphNodeGetType(nd, &t) == cudaSuccess && t == cudaGraphNodeTypeKernel) ++*kernels;
     }
-    e = cudaGraphInstantiate(out, g, 0);
+    // kernel nodes keep the priority of the stream they were captured on
+    e = cudaGraphInstantiateWithFlags(out, g, cudaGraphInstantiateFlagUseNodePriority);
     cudaGraphDestroy(g);
     if (e != cudaSuccess) return fail(PSML_ERR_CUDA, std::string("graph instantiate: ") + cudaGetErrorString(e));
     return PSML_OK;
