@@ -465,9 +465,10 @@ __global__ void __launch_bounds__(256) msb_chain_fused_kernel(MsbArgs<T> a, Chai
 
 // ---- the whole chain in one launch, one LANE PER PARTY ------------------------------------------
 // Lanes 2i and 2i+1 run the same element for party 0 and party 1.  Each round a lane computes its
-// party's masked words, writes them to that party's send buffer (the transcript a split deployment
-// would exchange) and obtains the peer's words with a lane-pair shuffle -- the co-resident form
-// of the opening (Eq. 5 / boolean e = x ^ a).  G, P stay in registers.  MODE 0: msb, 1: ReLU,
+// party's masked words and obtains the peer's words with a lane-pair shuffle -- the co-resident
+// form of the opening (Eq. 5 / boolean e = x ^ a); the messages never touch memory (the
+// per-round kernels, PSML_MSB_CHAIN=rounds, write them to the send buffers a split deployment
+// exchanges).  G, P and all dealer material stay in registers.  MODE 0: msb, 1: ReLU,
 // 2: Eq. 9 (lanes 0-15 run 8 elements of the first half [z + 1/2], lanes 16-31 the matching
 // elements of the second half [z - 1/2]; the final difference is a shuffle by 16).
 template <typename T>
@@ -498,7 +499,6 @@ __global__ void __launch_bounds__(256) msb_chain_pair_kernel(MsbArgs<T> a, Chain
         if (!valid) e = 0;
     }
     const T *mat = p ? a.mat.p[1] : a.mat.p[0];
-    T *msg = p ? a.msg.p[1] : a.msg.p[0];
     // Every load of the chain is data-independent: issue them all up front (one memory round trip
     // instead of one per protocol round -- the rounds' message stores would otherwise order them).
     T mt[2 * L][3];
@@ -521,7 +521,6 @@ __global__ void __launch_bounds__(256) msb_chain_pair_kernel(MsbArgs<T> a, Chain
     };
     // round 1: AND t = 0 on X = (x0, 0), Y = (0, x1)
     T m0 = (p == 0 ? x : (T)0) ^ M(0, 0), m1 = (p == 1 ? x : (T)0) ^ M(0, 1);
-    if (valid) { msg[e] = m0; msg[n + e] = m1; }
     T G = z_of(m0 ^ peer_of(m0), m1 ^ peer_of(m1), 0);
     T P = x;
 #pragma unroll
@@ -531,10 +530,6 @@ __global__ void __launch_bounds__(256) msb_chain_pair_kernel(MsbArgs<T> a, Chain
         const T g1 = P ^ M(t1, 0), h1 = (T)(G << k) ^ M(t1, 1);
         T g2 = 0, h2 = 0;
         if (j < L) { g2 = P ^ M(t2, 0); h2 = (T)(P << k) ^ M(t2, 1); }
-        if (valid) {
-            msg[e] = g1; msg[n + e] = h1;
-            if (j < L) { msg[2 * n + e] = g2; msg[3 * n + e] = h2; }
-        }
         const T z1 = z_of(g1 ^ peer_of(g1), h1 ^ peer_of(h1), t1);
         if (j < L) P = z_of(g2 ^ peer_of(g2), h2 ^ peer_of(h2), t2);
         G ^= z1;
@@ -542,7 +537,6 @@ __global__ void __launch_bounds__(256) msb_chain_pair_kernel(MsbArgs<T> a, Chain
     const T bit = ((x >> (l - 1)) & 1) ^ ((G >> (l - 2)) & 1);
     if (valid && SEL(o.msbB)) SEL(o.msbB)[e] = bit;
     const T cm = bit ^ rB;                    // B2A: c_i = msb_i ^ rB_i
-    if (valid) msg[e] = cm;
     const T c = cm ^ peer_of(cm);
     const T mA = (p == 0 ? c : (T)0) + ((T)1 - (T)2 * c) * rA;
     if (MODE == 0) {
@@ -553,7 +547,6 @@ __global__ void __launch_bounds__(256) msb_chain_pair_kernel(MsbArgs<T> a, Chain
     if (valid && SEL(o.drelu)) SEL(o.drelu)[e] = d;
     const T u = hu, v = hv;
     const T me = x - u, mf = d - v;           // Hadamard round: mask
-    if (valid) { SEL(o.mE)[e] = me; SEL(o.mF)[e] = mf; }
     const T E = me + peer_of(me), F = mf + peer_of(mf);
     const T r = (T)p * E * F + E * v + u * F + hz;
     if (MODE == 1) {
