@@ -94,7 +94,8 @@ __global__ void __launch_bounds__(256) open_kernel(OpenJobs<T> jobs) {
 }
 
 // ---------------------------------------------------------------------------------------------
-// two-segment GEMM
+// two-segment GEMM, grouped: up to SEG_MAX_JOBS independent products (e.g. gradW_l and gradin_l,
+// which consume the same delta) in one launch
 // ---------------------------------------------------------------------------------------------
 template <typename T>
 struct SegArgs {
@@ -107,6 +108,17 @@ struct SegArgs {
     int party[2];      // party index used by the truncation of slot p
     int64_t M, N, K;
     int trunc;
+    int nparty;        // 1 (split deployment) or 2 (co-resident)
+};
+
+constexpr int SEG_MAX_JOBS = 4;
+template <typename T>
+struct SegGroup {
+    SegArgs<T> j[SEG_MAX_JOBS];
+    int64_t tile_begin[SEG_MAX_JOBS + 1];   // prefix of tiles (x parties) per job
+    int64_t kps[SEG_MAX_JOBS];              // K slice per cluster rank, multiple of BK
+    int tiles_n[SEG_MAX_JOBS], tiles_m[SEG_MAX_JOBS];
+    int njobs, ks;
 };
 
 // epilogue adapter for cl_finish
@@ -139,17 +151,26 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 template <int N>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
-// grid (ceil(N/32), ceil(M/32), nparty * ks), cluster (1, 1, ks)
+// grid (total tiles, 1, ks), cluster (1, 1, ks)
 template <typename T>
-__global__ void __launch_bounds__(SegCfg::NT) seg_gemm_kernel(const __grid_constant__ SegArgs<T> a, int ks,
-                                                              int64_t k_per_split) {
+__global__ void __launch_bounds__(SegCfg::NT) seg_gemm_kernel(const __grid_constant__ SegGroup<T> g) {
     using C = SegCfg;
     __shared__ __align__(16) T smem[C::SMEM_WORDS];
     T *As = smem, *Bs = smem + C::STAGES * C::A_WORDS;   // As[s][mm][kk], Bs[s][kb][nn]
-    const int p = blockIdx.z / ks, split = blockIdx.z % ks;
-    const int64_t m0 = (int64_t)blockIdx.y * C::BM, n0 = (int64_t)blockIdx.x * C::BN;
+    const int64_t t = blockIdx.x;
+    int jb = 0;
+#pragma unroll
+    for (int q = 1; q < SEG_MAX_JOBS; ++q)
+        if (q < g.njobs && t >= g.tile_begin[q]) jb = q;
+    const SegArgs<T> &a = g.j[jb];
+    const int64_t tt = t - g.tile_begin[jb];
+    const int64_t per_party = (int64_t)g.tiles_m[jb] * g.tiles_n[jb];
+    const int p = (int)(tt / per_party);
+    const int64_t tp = tt - p * per_party;
+    const int64_t m0 = (tp / g.tiles_n[jb]) * C::BM, n0 = (tp % g.tiles_n[jb]) * C::BN;
+    const int ks = g.ks, split = blockIdx.z;
     const int64_t K = a.K, Kext = 2 * K;
-    const int64_t kbeg = (int64_t)split * k_per_split, kend = min(Kext, kbeg + k_per_split);
+    const int64_t kbeg = (int64_t)split * g.kps[jb], kend = min(Kext, kbeg + g.kps[jb]);
     const int nch = kend > kbeg ? (int)((kend - kbeg + C::BK - 1) / C::BK) : 0;
     const int tid = threadIdx.x;
     const T *Xp = a.X[p], *Vp = a.V[p];
@@ -157,8 +178,8 @@ __global__ void __launch_bounds__(SegCfg::NT) seg_gemm_kernel(const __grid_const
         const int st = c % C::STAGES;
         const int64_t k0 = kbeg + (int64_t)c * C::BK;
 #pragma unroll
-        for (int t = 0; t < C::A_WORDS / C::NT; ++t) {
-            const int idx = tid + t * C::NT, mm = idx / C::BK, kk = idx % C::BK;
+        for (int u = 0; u < C::A_WORDS / C::NT; ++u) {
+            const int idx = tid + u * C::NT, mm = idx / C::BK, kk = idx % C::BK;
             const int64_t m = m0 + mm, k = k0 + kk;
             const bool ok = m < a.M && k < kend;
             const int64_t mc = m < a.M ? m : a.M - 1, kc = k < kend ? k : kend - 1;
@@ -166,8 +187,8 @@ __global__ void __launch_bounds__(SegCfg::NT) seg_gemm_kernel(const __grid_const
             cp_async_elem<sizeof(T)>(As + st * C::A_WORDS + idx, src, ok);
         }
 #pragma unroll
-        for (int t = 0; t < C::B_WORDS / C::NT; ++t) {
-            const int idx = tid + t * C::NT, kb = idx / C::BN, nn = idx % C::BN;
+        for (int u = 0; u < C::B_WORDS / C::NT; ++u) {
+            const int idx = tid + u * C::NT, kb = idx / C::BN, nn = idx % C::BN;
             const int64_t k = k0 + kb, n = n0 + nn;
             const bool ok = n < a.N && k < kend;
             const int64_t kc = k < kend ? k : kend - 1, nc = n < a.N ? n : a.N - 1;
@@ -215,26 +236,48 @@ __global__ void __launch_bounds__(SegCfg::NT) seg_gemm_kernel(const __grid_const
     cl_finish<T, SegEpi<T>, C>(epi, p, m0, n0, ks, smem, acc);
 }
 
+// Launch 1..SEG_MAX_JOBS products as one grid; the cluster split ks is chosen for the group.
 template <typename T>
-psml_status launch_seg_gemm(const SegArgs<T> &a, int nparty, cudaStream_t stream, int sm_count) {
+psml_status launch_seg_group(const SegArgs<T> *jobs, int njobs, cudaStream_t stream, int sm_count) {
     using C = SegCfg;
-    const int64_t tiles = ((a.M + C::BM - 1) / C::BM) * ((a.N + C::BN - 1) / C::BN) * nparty;
-    const int ks = cl_splits(tiles, 2 * a.K, sm_count);
-    int64_t kps = (2 * a.K + ks - 1) / ks;
-    kps = ((kps + C::BK - 1) / C::BK) * C::BK;
+    if (njobs < 1 || njobs > SEG_MAX_JOBS) return fail(PSML_ERR_INVALID, "seg group: 1..4 jobs");
+    SegGroup<T> g{};
+    int64_t tiles = 0, kmax = 0;
+    double work = 0;
+    for (int q = 0; q < njobs; ++q) {
+        g.j[q] = jobs[q];
+        g.tiles_m[q] = (int)((jobs[q].M + C::BM - 1) / C::BM);
+        g.tiles_n[q] = (int)((jobs[q].N + C::BN - 1) / C::BN);
+        g.tile_begin[q] = tiles;
+        tiles += (int64_t)g.tiles_m[q] * g.tiles_n[q] * jobs[q].nparty;
+        kmax = std::max<int64_t>(kmax, 2 * jobs[q].K);
+        work += (double)jobs[q].M * jobs[q].N * 2 * jobs[q].K * jobs[q].nparty;
+    }
+    g.tile_begin[njobs] = tiles;
+    g.njobs = njobs;
+    g.ks = cl_splits(tiles, kmax, sm_count);
+    for (int q = 0; q < njobs; ++q) {
+        const int64_t kps = (2 * jobs[q].K + g.ks - 1) / g.ks;
+        g.kps[q] = ((kps + C::BK - 1) / C::BK) * C::BK;
+    }
     cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3((unsigned)((a.N + C::BN - 1) / C::BN), (unsigned)((a.M + C::BM - 1) / C::BM),
-                       (unsigned)(nparty * ks));
+    cfg.gridDim = dim3((unsigned)tiles, 1, (unsigned)g.ks);
     cfg.blockDim = dim3(C::NT);
     cfg.stream = stream;
     cudaLaunchAttribute attr[1];
     attr[0].id = cudaLaunchAttributeClusterDimension;
-    attr[0].val.clusterDim.x = 1; attr[0].val.clusterDim.y = 1; attr[0].val.clusterDim.z = (unsigned)ks;
+    attr[0].val.clusterDim.x = 1; attr[0].val.clusterDim.y = 1; attr[0].val.clusterDim.z = (unsigned)g.ks;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    ProfScope prof(PROF_GEMM, stream, (double)a.M * a.N * 2 * a.K * nparty);
-    PSML_CUDA_TRY(cudaLaunchKernelEx(&cfg, seg_gemm_kernel<T>, a, ks, kps));
+    ProfScope prof(PROF_GEMM, stream, work);
+    PSML_CUDA_TRY(cudaLaunchKernelEx(&cfg, seg_gemm_kernel<T>, g));
     return PSML_OK;
+}
+
+template <typename T>
+psml_status launch_seg_gemm(SegArgs<T> a, int nparty, cudaStream_t stream, int sm_count) {
+    a.nparty = nparty;
+    return launch_seg_group<T>(&a, 1, stream, sm_count);
 }
 
 template <typename T>

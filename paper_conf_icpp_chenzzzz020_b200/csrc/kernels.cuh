@@ -428,12 +428,34 @@ __global__ void eq9_open_kernel(CPair<T> mE, CPair<T> mF, CPair<T> U, CPair<T> V
 // next round opens them from there -- so the chain costs one launch instead of one per round.
 // (A split deployment exchanges the messages between rounds instead: msb_*_kernel per round.)
 // Eq. 9 pairs element e with e + n/2 so its final opening stays thread-local.
+// Opening of one consumer operand from a produced rows x cols matrix v (row-major, index e), used
+// by the fused training step (fused.cuh): dst index di = e (trans = 0) or (e % cols) * rows +
+// e / cols (the consumer reads v^T); E[di] = (v_0 - M_0[di]) + (v_1 - M_1[di]) and, for an A side,
+// X1[di] = E[di] + M_1[di].
+template <typename T>
+struct Emit {
+    const T *M[2];
+    T *E, *X1;
+    int64_t rows, cols;
+    int trans;
+};
+template <typename T>
+struct Emits {
+    Emit<T> e[2];
+    int n;
+};
+template <typename T>
+__device__ __forceinline__ int64_t emit_index(const Emit<T> &em, int64_t e) {
+    return em.trans ? (e % em.cols) * em.rows + e / em.cols : e;
+}
+
 template <typename T>
 struct ChainOut {
     Pair<T> msbA, msbB, drelu, y, delta;
     CPair<T> U, V, Z, Ysub;
     Pair<T> mE, mF;
     int what;
+    Emits<T> em;   // consumer opens of y (ReLU) / delta (Eq. 9); lane-pair kernel only
 };
 
 template <typename T>
@@ -514,6 +536,27 @@ __global__ void __launch_bounds__(256) msb_chain_pair_kernel(MsbArgs<T> a, Chain
     T hu = 0, hv = 0, hz = 0, ysub = 0;
     if (MODE != 0) { hu = SEL(o.U)[e]; hv = SEL(o.V)[e]; hz = SEL(o.Z)[e]; }
     if (MODE == 2 && !second && SEL(o.Ysub)) ysub = SEL(o.Ysub)[e];
+    T emk[2] = {0, 0};
+    int64_t edi[2] = {0, 0};
+#pragma unroll
+    for (int q = 0; q < 2; ++q)
+        if (q < o.em.n && (MODE != 2 || !second)) {
+            edi[q] = emit_index(o.em.e[q], e);
+            emk[q] = o.em.e[q].M[p][edi[q]];
+        }
+    // consumer opens of this lane pair's value v (both parties: v here, the peer's by shuffle)
+    auto emit = [&](T v, bool ok) {
+#pragma unroll
+        for (int q = 0; q < 2; ++q) {
+            if (q >= o.em.n) break;
+            const T part = v - emk[q];
+            const T E = part + peer_of(part);
+            if (ok) {
+                if (p == 0) o.em.e[q].E[edi[q]] = E;
+                else if (o.em.e[q].X1) o.em.e[q].X1[edi[q]] = E + emk[q];
+            }
+        }
+    };
     auto M = [&](int t, int w) -> T { return mt[t][w]; };
     auto z_of = [&](T ee, T ff, int t) -> T {
         T r = (ee & M(t, 1)) ^ (M(t, 0) & ff) ^ M(t, 2);
@@ -550,15 +593,18 @@ __global__ void __launch_bounds__(256) msb_chain_pair_kernel(MsbArgs<T> a, Chain
     const T E = me + peer_of(me), F = mf + peer_of(mf);
     const T r = (T)p * E * F + E * v + u * F + hz;
     if (MODE == 1) {
-        if (valid) SEL(o.y)[e] = r;
+        if (valid && SEL(o.y)) SEL(o.y)[e] = r;
+        emit(r, valid);
         return;
     }
     const T r2 = (T)__shfl_xor_sync(0xffffffffu, (unsigned long long)r, 16);
+    const T out = r - r2;                     // ReLU(z + 1/2) - ReLU(z - 1/2)
+    const T dl = out - ysub;
     if (valid && !second) {
-        const T out = r - r2;                 // ReLU(z + 1/2) - ReLU(z - 1/2)
         if (SEL(o.y)) SEL(o.y)[e] = out;
-        if (SEL(o.delta)) SEL(o.delta)[e] = out - ysub;
+        if (SEL(o.delta)) SEL(o.delta)[e] = dl;
     }
+    emit(dl, valid && !second);
 }
 
 #undef SEL

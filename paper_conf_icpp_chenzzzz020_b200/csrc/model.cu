@@ -18,6 +18,7 @@
 
 #include "engine.h"
 #include "dealer_fused.cuh"
+#include "fused.cuh"
 
 namespace psml {
 
@@ -36,6 +37,17 @@ static bool fused_open() {
     if (m < 0) {
         const char *e = getenv("PSML_OPEN");
         m = (e && e[0] == 'f') ? 1 : 0;
+    }
+    return m == 1;
+}
+
+// Fused co-resident training step (fused.cuh): producers open their consumers' operands
+// (default) or one open pass per product (PSML_FUSE=0); bit-identical (tested).
+static bool fuse_enabled() {
+    static int m = -1;
+    if (m < 0) {
+        const char *e = getenv("PSML_FUSE");
+        m = (e && e[0] == '0') ? 0 : 1;
     }
     return m == 1;
 }
@@ -71,6 +83,10 @@ struct DealItem {
     Buf U, V, Z, mat;
 };
 
+struct OpenBuf {    // opened operands of one matrix product (fused step): E, X_1 (M x K), F (K x N)
+    T *E = nullptr, *X1 = nullptr, *F = nullptr;
+};
+
 struct DealPlan {   // fused dealer of one pool (full or inference-only)
     PrgJob *prg = nullptr;
     int n_prg = 0;
@@ -102,6 +118,7 @@ struct psml_model_s {
     // run concurrently with the online phase of step s (offline/online pipelining).
     std::vector<psml::DealItem> items[2];
     psml::DealPlan plan[2][2];         // [pool][infer_only]
+    std::vector<psml::OpenBuf> ob;     // per item index (fused step; empty when not eligible)
     int pool = 0;                      // pool the online phase is reading
     psml::T *ws = nullptr;             // online workspace
     int64_t ws_words = 0;
@@ -581,6 +598,189 @@ static psml_status backward(psml_model_s *m, cudaStream_t s) {
     return PSML_OK;
 }
 
+// ------------------------------------------------------------------------------------------------
+// fused co-resident training step (fused.cuh): MLP / linear / logistic regression
+// ------------------------------------------------------------------------------------------------
+static int item_index(const psml_model_s *m, int layer, int op, int slot) {
+    for (size_t k = 0; k < m->items[0].size(); ++k) {
+        const DealItem &it = m->items[0][k];
+        if (it.layer == layer && it.op == op && it.slot == slot) return (int)k;
+    }
+    return -1;
+}
+
+static bool fused_eligible(const psml_model_s *m) {
+    if (m->d.kind == PSML_CNN || m->nl > UPD_MAX_LAYERS || (int)m->ob.size() != (int)m->items[0].size()) return false;
+    return fuse_enabled() && chain_mode() == 0;
+}
+
+static bool fused_shapes_ok(const psml_model_s *m) {
+    if (m->d.kind == PSML_CNN || m->nl > UPD_MAX_LAYERS) return false;
+    for (auto &it : m->items[0])
+        if (it.kind == IT_MATRIX && m->ctx->use_tc(it.M, 2 * it.K, it.N)) return false;
+    return true;
+}
+
+static psml_status alloc_open_bufs(psml_model_s *m) {
+    m->ob.assign(m->items[0].size(), OpenBuf{});
+    for (size_t k = 0; k < m->items[0].size(); ++k) {
+        const DealItem &it = m->items[0][k];
+        if (it.kind != IT_MATRIX) continue;
+        PSML_TRY(dalloc(m, &m->ob[k].E, it.M * it.K));
+        PSML_TRY(dalloc(m, &m->ob[k].X1, it.M * it.K));
+        PSML_TRY(dalloc(m, &m->ob[k].F, it.K * it.N));
+    }
+    return PSML_OK;
+}
+
+static psml_status fused_forward_backward(psml_model_s *m, const T *const X[2], const T *const Y[2], cudaStream_t s) {
+    const int F = m->ctx->ring.frac_bits;
+    const int nl = m->nl;
+    const int64_t B = m->B;
+    auto &items = m->items[m->pool];
+    auto idx = [&](int l, int op, int slot = 0) { return item_index(m, l, op, slot); };
+    for (int l = 0; l < nl; ++l)
+        if (idx(l, OP_FWD) < 0 || idx(l, OP_GRADW) < 0 || (l > 0 && idx(l, OP_GRADIN) < 0))
+            return fail(PSML_ERR_STATE, "fused step: missing triplet");
+    m->act[0].p[0] = (T *)X[0];
+    m->act[0].p[1] = (T *)X[1];
+    auto seg = [&](int l, int op, T *C0, T *C1, int trunc) {
+        const int k = idx(l, op);
+        const DealItem &it = items[k];
+        const OpenBuf &o = m->ob[k];
+        SegArgs<T> a{};
+        a.X[0] = it.U.p[0]; a.X[1] = o.X1; a.E = o.E; a.F = o.F;
+        for (int p = 0; p < 2; ++p) { a.V[p] = it.V.p[p]; a.Z[p] = it.Z.p[p]; a.party[p] = p; }
+        a.C[0] = C0; a.C[1] = C1;
+        a.M = it.M; a.N = it.N; a.K = it.K; a.trunc = trunc; a.nparty = 2;
+        return a;
+    };
+    // A side of product (l, op): mask U, outputs E, X_1;  B side: mask V, output F
+    auto emitA = [&](int l, int op, int64_t rows, int64_t cols, int trans) {
+        const int k = idx(l, op);
+        Emit<T> e{};
+        e.M[0] = items[k].U.p[0]; e.M[1] = items[k].U.p[1];
+        e.E = m->ob[k].E; e.X1 = m->ob[k].X1; e.rows = rows; e.cols = cols; e.trans = trans;
+        return e;
+    };
+    auto emitB = [&](int l, int op, int64_t rows, int64_t cols) {
+        const int k = idx(l, op);
+        Emit<T> e{};
+        e.M[0] = items[k].V.p[0]; e.M[1] = items[k].V.p[1];
+        e.E = m->ob[k].F; e.X1 = nullptr; e.rows = rows; e.cols = cols; e.trans = 0;
+        return e;
+    };
+    // 1. step-start opens: the input batch and every weight matrix
+    {
+        OpenList<T> L{};
+        int n = 0;
+        int64_t tiles = 0;
+        auto add = [&](const T *s0, const T *s1, const T *m0, const T *m1, T *open, T *x, int64_t rows, int64_t cols,
+                       int trans) {
+            OpenJob<T> &j = L.j[n];
+            j.src[0] = s0; j.src[1] = s1; j.mask[0] = m0; j.mask[1] = m1;
+            j.open = open; j.x = x; j.xmask = x ? m1 : nullptr; j.scale = 1;
+            j.rows = rows; j.cols = cols; j.trans = trans;
+            L.tile_begin[n] = tiles;
+            tiles += ((rows + 31) / 32) * ((cols + 31) / 32);
+            ++n;
+        };
+        {
+            const int k = idx(0, OP_FWD);
+            add(X[0], X[1], items[k].U.p[0], items[k].U.p[1], m->ob[k].E, m->ob[k].X1, B, m->dims[0], 0);
+            const int g = idx(0, OP_GRADW);   // op(A) = X^T (d_0 x B), X stored B x d_0
+            add(X[0], X[1], items[g].U.p[0], items[g].U.p[1], m->ob[g].E, m->ob[g].X1, m->dims[0], B, 1);
+        }
+        for (int l = 0; l < nl; ++l) {
+            const int k = idx(l, OP_FWD);
+            add(m->W[l].p[0], m->W[l].p[1], items[k].V.p[0], items[k].V.p[1], m->ob[k].F, nullptr, m->dims[l],
+                m->dims[l + 1], 0);
+            if (l > 0) {   // op(B) = W_l^T (d_{l+1} x d_l), W_l stored d_l x d_{l+1}
+                const int g = idx(l, OP_GRADIN);
+                add(m->W[l].p[0], m->W[l].p[1], items[g].V.p[0], items[g].V.p[1], m->ob[g].F, nullptr,
+                    m->dims[l + 1], m->dims[l], 1);
+            }
+        }
+        L.n = n;
+        L.tile_begin[n] = tiles;
+        ProfScope prof(PROF_MASK, s, 0.0);
+        open_list_kernel<T><<<(unsigned)tiles, dim3(32, 8), 0, s>>>(L);
+        PSML_LAUNCH_CHECK();
+    }
+    // 2. forward
+    T *yo[2] = {m->yhat.p[0], m->yhat.p[1]};
+    for (int l = 0; l < nl; ++l) {
+        SegArgs<T> a = seg(l, OP_FWD, m->z[l].p[0], m->z[l].p[1], F);
+        PSML_TRY(launch_seg_group<T>(&a, 1, s, m->ctx->sm_count));
+        const int64_t w = m->dims[l + 1];
+        if (l < nl - 1) {
+            Emits<T> em{};
+            em.e[0] = emitA(l + 1, OP_FWD, B, w, 0);
+            em.e[1] = emitA(l + 1, OP_GRADW, B, w, 1);
+            em.n = 2;
+            DealItem *mat = find_item(m, l, OP_RELU_MSB, 0), *h = find_item(m, l, OP_HADAMARD, 0);
+            if (!mat || !h) return fail(PSML_ERR_STATE, "missing ReLU material");
+            PSML_TRY(msb_chain<T>(m->z[l].cp(), mat->n, mat->mat.cp(), 0, 0, 1, nullptr, nullptr, m->drelu[l].pp(),
+                                  h->U.cp(), h->V.cp(), h->Z.cp(), m->act[l + 1].pp(), nullptr, nullptr, m->ws, s,
+                                  &em));
+        } else {
+            Emits<T> em{};
+            em.e[0] = emitB(l, OP_GRADW, B, w);
+            em.n = 1;
+            if (l > 0) { em.e[1] = emitA(l, OP_GRADIN, B, w, 0); em.n = 2; }
+            if (is_eq9_out(m)) {
+                DealItem *mat = find_item(m, l, OP_EQ9_MSB, 0), *h = find_item(m, l, OP_HADAMARD, 2);
+                if (!mat || !h) return fail(PSML_ERR_STATE, "missing Eq. 9 material");
+                const T half = (T)1 << (F - 1);
+                PSML_TRY(msb_chain<T>(m->z[l].cp(), mat->n, mat->mat.cp(), 1, half, 2, nullptr, nullptr, nullptr,
+                                      h->U.cp(), h->V.cp(), h->Z.cp(), yo, Y, m->delta.pp(), m->ws, s, &em));
+            } else {
+                DeltaFused<T> d{};
+                for (int p = 0; p < 2; ++p) {
+                    d.z[p] = m->z[l].p[p]; d.Y[p] = Y[p]; d.yhat[p] = yo[p]; d.delta[p] = m->delta.p[p];
+                }
+                d.n = B * w;
+                d.em = em;
+                delta_fused_kernel<T><<<ew_grid(d.n), EW_THREADS, 0, s>>>(d);
+                PSML_LAUNCH_CHECK();
+            }
+        }
+    }
+    // 3. backward: gradW_l and gradin_l in one launch, then the backprop Hadamard opens delta_{l-1}
+    T *g[2];
+    for (int l = nl - 1; l >= 0; --l) {
+        gradp(m, l, g);
+        SegArgs<T> jobs[2];
+        jobs[0] = seg(l, OP_GRADW, g[0], g[1], 0);
+        if (l > 0) jobs[1] = seg(l, OP_GRADIN, m->tmp.p[0], m->tmp.p[1], F);
+        PSML_TRY(launch_seg_group<T>(jobs, l > 0 ? 2 : 1, s, m->ctx->sm_count));
+        if (l > 0) {
+            DealItem *h = find_item(m, l - 1, OP_HADAMARD, 1);
+            if (!h) return fail(PSML_ERR_STATE, "missing Hadamard triplet");
+            const int64_t w = m->dims[l];
+            HadFused<T> hf{};
+            for (int p = 0; p < 2; ++p) {
+                hf.a[p] = m->tmp.p[p]; hf.b[p] = m->drelu[l - 1].p[p];
+                hf.U[p] = h->U.p[p]; hf.V[p] = h->V.p[p]; hf.Z[p] = h->Z.p[p]; hf.c[p] = m->delta.p[p];
+            }
+            hf.n = B * w;
+            hf.em.e[0] = emitB(l - 1, OP_GRADW, B, w);
+            hf.em.n = 1;
+            if (l - 1 > 0) { hf.em.e[1] = emitA(l - 1, OP_GRADIN, B, w, 0); hf.em.n = 2; }
+            ProfScope prof(PROF_HAD, s, 0.0);
+            had_fused_kernel<T><<<ew_grid(hf.n), EW_THREADS, 0, s>>>(hf);
+            PSML_LAUNCH_CHECK();
+        }
+    }
+    return PSML_OK;
+}
+
+static psml_status forward_backward(psml_model_s *m, const T *const X[2], const T *const Y[2], cudaStream_t s) {
+    if (fused_eligible(m)) return fused_forward_backward(m, X, Y, s);
+    PSML_TRY(forward(m, X, Y, nullptr, s));
+    return backward(m, s);
+}
+
 }  // namespace psml
 
 using namespace psml;
@@ -678,6 +878,7 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
     PSML_TRY(alloc_items(mp, m->items[1]));
     for (int pl = 0; pl < 2; ++pl)
         for (int inf = 0; inf < 2; ++inf) PSML_TRY(build_plan(mp, pl, inf != 0));
+    if (fused_shapes_ok(mp)) PSML_TRY(alloc_open_bufs(mp));
     m->dws_words = dws_need(mp);
     PSML_TRY(dalloc(mp, &m->dws, m->dws_words));
     {
@@ -769,8 +970,7 @@ psml_status psml_train_forward_backward(psml_model m, const void *const X[2], co
         return fail(PSML_ERR_STATE, "psml_model_deal(step_id, infer_only=0) must precede the step");
     cudaStream_t s = (cudaStream_t)stream;
     m->pool = pool;
-    PSML_TRY(forward(m, (const T *const *)X, (const T *const *)Y, nullptr, s));
-    PSML_TRY(backward(m, s));
+    PSML_TRY(forward_backward(m, (const T *const *)X, (const T *const *)Y, s));
     m->grads_ready = true;
     return PSML_OK;
 }
@@ -798,6 +998,23 @@ psml_status psml_train_apply_update(psml_model m, int32_t extra_shift, psml_stre
     const int f = m->ctx->ring.frac_bits;
     const int s_grad = 2 * f + m->d.lr_shift - m->d.master_frac_bits + extra_shift;
     const int s_fwd = m->d.master_frac_bits - f;
+    if (m->nl <= UPD_MAX_LAYERS) {   // every layer in one launch
+        UpdateAll<T> u{};
+        int64_t tot = 0;
+        for (int l = 0; l < m->nl; ++l) {
+            T *g[2];
+            gradp(m, l, g);
+            for (int p = 0; p < 2; ++p) { u.Wm[l][p] = m->Wm[l].p[p]; u.W[l][p] = m->W[l].p[p]; u.g[l][p] = g[p]; }
+            u.begin[l] = tot;
+            tot += m->rows[l] * m->cols[l];
+        }
+        u.begin[m->nl] = tot;
+        u.nl = m->nl; u.s_grad = s_grad; u.s_fwd = s_fwd;
+        update_all_kernel<T><<<ew_grid(tot), EW_THREADS, 0, s>>>(u);
+        PSML_LAUNCH_CHECK();
+        m->grads_ready = false;
+        return PSML_OK;
+    }
     for (int l = 0; l < m->nl; ++l) {
         const int64_t n = m->rows[l] * m->cols[l];
         T *g[2];
@@ -850,8 +1067,7 @@ static psml_status capture_one(psml_model_s *m, int pool, const T *const X[2], c
         st = deal_pool(m, pool, 0, false, s);
     }
     m->pool = pool;
-    if (st == PSML_OK) st = forward(m, X, Y, nullptr, on);
-    if (st == PSML_OK) st = backward(m, on);
+    if (st == PSML_OK) st = forward_backward(m, X, Y, on);
     if (st == PSML_OK && (flags & 2)) {
         m->grads_ready = true;
         st = psml_train_apply_update(m, 0, (psml_stream)on);

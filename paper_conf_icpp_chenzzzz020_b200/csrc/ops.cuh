@@ -203,8 +203,10 @@ template <typename T>
 psml_status msb_chain(const T *const x[2], int64_t n, const T *const mat[2], int mode, T half,
                       int what, T *const msbA[2], T *const msbB[2], T *const drelu[2],
                       const T *const U[2], const T *const V[2], const T *const Z[2], T *const y[2],
-                      const T *const Ysub[2], T *const delta[2], T *ws, cudaStream_t s) {
+                      const T *const Ysub[2], T *const delta[2], T *ws, cudaStream_t s,
+                      const Emits<T> *em = nullptr) {
     const int l = 8 * (int)sizeof(T);
+    if (em && em->n && chain_mode() != 0) return fail(PSML_ERR_UNSUPPORTED, "operand emits need the lane-pair chain");
     MsbArgs<T> a;
     a.x = CPair<T>{{x[0], x[1]}};
     a.mat = CPair<T>{{mat[0], mat[1]}};
@@ -229,6 +231,8 @@ psml_status msb_chain(const T *const x[2], int64_t n, const T *const mat[2], int
     o.mE = mE;
     o.mF = mF;
     o.what = what;
+    o.em.n = 0;
+    if (em) o.em = *em;
     if (chain_mode() == 0) {   // one launch; lane pair = (party 0, party 1) of one element
         const int64_t threads = what == 2 ? ((n / 2 + 7) / 8) * 32 : 2 * n;
         const int blocks = (int)((threads + EW_THREADS - 1) / EW_THREADS);

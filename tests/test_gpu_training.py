@@ -130,13 +130,14 @@ def test_cnn_one_epoch_against_fp64(T):
 def test_explicit_mask_round_matches_fused_open():
     """PSML_OPEN=fused (mask round fused into the GEMM loads), PSML_MSB_CHAIN=rounds (one kernel
     per protocol round) and PSML_DEAL=items (one dealer launch group per item instead of the two
-    fused dealer launches) and PSML_SIMT=small (16 x 16 one-output-per-thread GEMM instead of the
-    cluster split-K kernel) reproduce the oracle exactly, like the defaults."""
+    fused dealer launches), PSML_SIMT=small (16 x 16 one-output-per-thread GEMM instead of the
+    cluster split-K kernel) and PSML_FUSE=0 (one open pass per product instead of producer-side
+    opens) reproduce the oracle exactly, like the defaults."""
     import os
     import subprocess
     import sys
     env = dict(os.environ, PSML_OPEN="fused", PSML_MSB_CHAIN="rounds", PSML_DEAL="items",
-               PSML_SIMT="small")
+               PSML_SIMT="small", PSML_FUSE="0")
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
     r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu", "-k",
                         "training_bitexact_vs_oracle or graph_replay", os.path.join(root, "tests", "test_gpu_training.py")],
