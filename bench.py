@@ -49,6 +49,10 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--task", default="mlp", choices=sorted(WORKLOADS),
                     help="headline is mlp (BASELINE metric); others are secondary configs")
+    ap.add_argument("--deployment", default="coresident", choices=["coresident", "split"],
+                    help="coresident: both parties of a pair on one GPU (default); split: party 0 "
+                         "and party 1 on different GPUs (ranks k and k + N/2), every opening "
+                         "round exchanged over NCCL (SURVEY 8(e))")
     a = ap.parse_args()
     global TASK, WORKLOAD
     TASK, WORKLOAD = a.task, WORKLOADS[a.task]
@@ -316,6 +320,96 @@ def bench_ours(args):
     return result, tr, world, rank
 
 
+def bench_split(args):
+    """Split deployment: N/2 party pairs, pair k = (rank k: party 0, rank k + N/2: party 1); each
+    pair trains on its own 128 rows; every opening is an NCCL exchange between the pair's GPUs
+    (library-owned communicator); each party all-reduces its gradient share over its N/2 ranks."""
+    import torch
+    import torch.distributed as dist
+
+    import synth
+    from paper_conf_icpp_chenzzzz020_b200 import build, psml
+    from paper_conf_icpp_chenzzzz020_b200.parallel import make_transport, pair_layout
+    from paper_conf_icpp_chenzzzz020_b200.train import PartyTrainer
+
+    build.build()
+    world, rank, local = dist_setup(args)
+    party, pair, peer = pair_layout(world)(rank)
+    half = world // 2
+    groups = [dist.new_group(list(range(q * half, (q + 1) * half))) for q in range(2)]
+    dev = torch.device("cuda", local)
+    K, W = args.steps, args.warmup
+    xp = make_transport(party, peer)
+    tr = PartyTrainer(TASK, synth.init_weights(TASK), party, xp, batch=BATCH, pair_id=pair)
+    nb = K + W
+    Xs, Ys = [], []
+    for s in range(nb):
+        X, Y = synth.batch(TASK, s, BATCH, pair=pair, n_pairs=half)
+        Xs.append(torch.from_numpy(X).to(dev))
+        Ys.append(torch.from_numpy(Y).to(dev))
+    Xh = [x.cpu().pin_memory() for x in Xs]
+    Yh = [y.cpu().pin_memory() for y in Ys]
+    stream = torch.cuda.current_stream()
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+
+    def step(s, X, Y):
+        X_i, Y_i = tr.share_batch(X, Y, s)
+        tr.step_party(X_i, Y_i, s, dp_group=groups[party], dp_world=half)
+
+    def timed(fn, n, base):
+        dist.barrier()
+        torch.cuda.synchronize()
+        tot = 0.0
+        for i in range(n):
+            flush.zero_()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            fn(base + i)
+            b.record(stream)
+            b.synchronize()
+            tot += a.elapsed_time(b) / 1e3
+        dist.barrier()
+        return max_over_ranks(tot, world)
+
+    for s in range(W):
+        step(s, Xs[s], Ys[s])
+    torch.cuda.synchronize()
+    b0, x0 = xp.stats()
+    l0 = psml.kernel_launch_count()
+    with ClockSampler(local) as clk:
+        t_dev = timed(lambda s: step(s, Xs[s], Ys[s]), K, W)
+    launches = psml.kernel_launch_count() - l0
+    b1, x1 = xp.stats()
+    out_host = torch.empty(BATCH * Ys[0].shape[1], dtype=torch.uint64).pin_memory()
+
+    def e2e(s):
+        i = (s - W - K) % nb
+        step(s, Xh[i].to(dev, non_blocking=True), Yh[i].to(dev, non_blocking=True))
+        ptrs = tr.model.output()
+        from paper_conf_icpp_chenzzzz020_b200.train import _wrap_device_ptr
+        out_host.copy_(_wrap_device_ptr(ptrs[party], ptrs[2], "<u8"), non_blocking=True)
+    t_e2e = timed(e2e, K, W + K)
+    samples = BATCH * K * half
+    return {
+        "metric": METRIC, "value": samples / t_dev, "unit": "samples/s", "n_gpus": world,
+        "steps": K, "warmup": W, "ms_per_step": 1e3 * t_dev / K, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "u64",
+        "data": "synthetic (MNIST-shaped 784 features, 81% zeros; teacher labels)",
+        "config": {"workload": WORKLOAD, "deployment": "split (one party per GPU)",
+                   "global_batch": BATCH * half, "per_pair_batch": BATCH, "pairs": half,
+                   "ring": "Z_2^64, 13 fractional bits", "parallelism": f"{half} pairs x 2 parties",
+                   "l2": "256 MiB flush between timed steps (outside the events)",
+                   "step": "client share, dealer (each party's half), online step with one "
+                           "exchange per opening round, gradient all-reduce per party, update"},
+        "exchanges_per_step": (x1 - x0) / K, "bytes_sent_per_step_per_party": (b1 - b0) / K,
+        "e2e": {"value": samples / t_e2e, "unit": "samples/s",
+                "h2d_bytes_per_step": Xh[0].numel() * 8 + Yh[0].numel() * 8,
+                "d2h_bytes_per_step": out_host.numel() * 8},
+        "gpu_launches": int(launches), "clocks": clk.summary(),
+        "roofline": None,
+    }, rank
+
+
 def measured_peaks():
     try:
         return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
@@ -443,6 +537,11 @@ def main():
         out = bench_reference(args)
         if out is not None:
             print(json.dumps(out), flush=True)
+        return
+    if args.deployment == "split":
+        result, rank = bench_split(args)
+        if rank == 0:
+            print(json.dumps(result), flush=True)
         return
     result, tr, world, rank = bench_ours(args)
     if TASK != "mlp":

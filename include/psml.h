@@ -49,7 +49,8 @@ typedef enum {
     PSML_ERR_UNSUPPORTED = 4, /* configuration not built (e.g. no sm_100 device)              */
     PSML_ERR_CUDA = 5,        /* a CUDA runtime/driver call or kernel launch failed           */
     PSML_ERR_NOMEM = 6,       /* device allocation failed                                     */
-    PSML_ERR_STATE = 7        /* object used in the wrong state (e.g. step without deal)      */
+    PSML_ERR_STATE = 7,       /* object used in the wrong state (e.g. step without deal)      */
+    PSML_ERR_NCCL = 8         /* a transport exchange (NCCL call or host callback) failed     */
 } psml_status;
 
 /* The ring Z_{2^l} and the fixed-point scale (SecureML: frac_bits = 13).  DESIGN.md R3. */
@@ -294,6 +295,53 @@ psml_status psml_model_graph_nodes(psml_model model, int64_t *n);
  * psml_model_deal(step_id, infer_only=1) (or a full deal) for the same step_id. */
 psml_status psml_secure_infer(psml_model model, const void *const X[2], uint32_t step_id,
                               void *const Yhat[2], psml_stream stream);
+
+/* ------------------------------------------------------------------------------------------ */
+/* Split deployment: ONE party per process / GPU (Fig. 1b L55-L61: two non-colluding  */
+/* servers; L65 "compute E and F via communication").  Every opening of the training step --   */
+/* the E/F of each Beaver product (Eq. 5), the boolean AND rounds of the MSB chain, the daBit  */
+/* B2A word and the Hadamard E/F (R9) -- becomes one symmetric exchange of the        */
+/* party's masked message through a transport.  Shares and opened values are bit-identical to */
+/* the co-resident engine (same kernels, restricted to one party).                              */
+/* ------------------------------------------------------------------------------------------ */
+typedef struct psml_xport_s *psml_xport;
+
+/* Host callback transport (any backend; used for host-staged gloo).  Must send, for every
+ * k < n, `bytes[k]` bytes at device address send[k] to the peer and receive the peer's
+ * same-sized message into device address recv[k], ordered after the work already enqueued on
+ * `stream` and before work enqueued after it returns (synchronise the stream first).  Returns 0
+ * on success; non-zero makes the step fail with PSML_ERR_NCCL. */
+typedef int32_t (*psml_exchange_fn)(void *user, int32_t n, void *const *send, void *const *recv,
+                                    const int64_t *bytes, psml_stream stream);
+
+/* 128-byte NCCL unique id (created by one party, broadcast by the caller, e.g. over a
+ * torch.distributed process group). */
+psml_status psml_nccl_unique_id(uint8_t uid[128]);
+/* NCCL transport: the library creates and owns a 2-rank communicator (this party = `rank`,
+ * the peer = 1 - rank) on the current device; exchanges are grouped ncclSend/ncclRecv on the
+ * step's stream (stream-ordered, no host synchronisation; NVLink P2P between GPUs). */
+psml_status psml_xport_nccl_create(const uint8_t uid[128], int32_t rank, psml_xport *out);
+psml_status psml_xport_callback_create(psml_exchange_fn fn, void *user, psml_xport *out);
+psml_status psml_xport_destroy(psml_xport x);
+/* One symmetric exchange of n device buffers (what every opening round does). */
+psml_status psml_xport_exchange(psml_xport x, int32_t n, const void *const *send, void *const *recv,
+                                const int64_t *bytes, psml_stream stream);
+/* Bytes and exchanges issued through this transport so far (accounting for bench.py). */
+psml_status psml_xport_stats(psml_xport x, int64_t *bytes_sent, int64_t *exchanges);
+
+/* Party `party`'s half of one training step (LINREG / LOGREG / MLP; PSML_ERR_UNSUPPORTED for
+ * CNN): X_i: batch x d_0, Y_i: batch x d_L, this party's shares (device).  The model's dealer
+ * pool must hold the step's material (psml_model_deal; in this simulation each party's process
+ * runs the dealer and reads only its own half -- a deployment ships it from the client).
+ * Leaves this party's untruncated weight-gradient share in psml_model_grads()[party] and its
+ * prediction share in psml_model_output; then psml_party_apply_update updates this party's
+ * master/forward weight shares (extra_shift as psml_train_apply_update).  Both parties must
+ * call with the same step_id; every exchange is collective between them. */
+psml_status psml_party_forward_backward(psml_model model, int32_t party, psml_xport x,
+                                        const void *X_i, const void *Y_i, uint32_t step_id,
+                                        psml_stream stream);
+psml_status psml_party_apply_update(psml_model model, int32_t party, int32_t extra_shift,
+                                    psml_stream stream);
 
 #ifdef __cplusplus
 }

@@ -6,7 +6,7 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libpsml.so")
-SOURCES = ["engine.cu", "model.cu", "gemm_tc.cu", "codec.cu"]
+SOURCES = ["engine.cu", "model.cu", "gemm_tc.cu", "codec.cu", "xport.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "--expt-relaxed-constexpr", "-Xcompiler", "-fPIC,-fvisibility=hidden", "-Xptxas", "-v"]
@@ -44,7 +44,7 @@ def build(force=False, verbose=False, jobs=4):
     if failed:
         raise RuntimeError("libpsml build failed")
     cmd = [NVCC, "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-o", LIB + ".tmp"] + objs \
-        + ["-lcudart_static", "-ldl", "-lrt", "-lpthread"]
+        + ["-lcudart_static", "-lnccl", "-ldl", "-lrt", "-lpthread"]
     subprocess.check_call(cmd)
     os.replace(LIB + ".tmp", LIB)
     return LIB

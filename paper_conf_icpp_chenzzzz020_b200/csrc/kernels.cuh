@@ -224,10 +224,11 @@ __global__ void mask_kernel(MaskJobs<T> jobs) {
 // ---------------------------------------------------------------------------------------------
 template <typename T>
 __global__ void hadamard_mask_kernel(CPair<T> A, CPair<T> B, CPair<T> U, CPair<T> V, int64_t n,
-                                     Pair<T> mE, Pair<T> mF) {
+                                     Pair<T> mE, Pair<T> mF, int only = -1) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
 #pragma unroll
         for (int p = 0; p < 2; ++p) {
+            if (only >= 0 && p != only) continue;
             mE.p[p][i] = A.p[p][i] - U.p[p][i];
             mF.p[p][i] = B.p[p][i] - V.p[p][i];
         }
@@ -250,7 +251,12 @@ struct MsbArgs {
     int mode;
     T half;            // 2^(f-1) for mode 1
     int L, l;
+    // -1: co-resident (both parties).  0 / 1: split deployment -- this process is party `only`;
+    // msg.p[only] is its send buffer and msg.p[1 - only] the peer's received words (same layout).
+    int only = -1;
 };
+#define PSML_PARTY_SKIP(a, p) \
+    if ((a).only >= 0 && (p) != (a).only) continue;
 
 template <typename T>
 __device__ __forceinline__ T msb_input(const MsbArgs<T> &a, int p, int64_t e) {
@@ -272,6 +278,7 @@ __device__ __forceinline__ void and_open(const MsbArgs<T> &a, int64_t e, int w, 
     const T ff = a.msg.p[0][(int64_t)(w + 1) * a.n + e] ^ a.msg.p[1][(int64_t)(w + 1) * a.n + e];
 #pragma unroll
     for (int p = 0; p < 2; ++p) {
+        PSML_PARTY_SKIP(a, p)
         T r = (ee & mat_ptr(a, p, t, 1)[e]) ^ (mat_ptr(a, p, t, 0)[e] & ff) ^ mat_ptr(a, p, t, 2)[e];
         z[p] = p == 1 ? (T)(r ^ (ee & ff)) : r;
     }
@@ -283,6 +290,7 @@ template <typename T>
 __device__ __forceinline__ void msb_round0_body(const MsbArgs<T> &a, int64_t e) {
 #pragma unroll
     for (int p = 0; p < 2; ++p) {
+        PSML_PARTY_SKIP(a, p)
         T x = msb_input(a, p, e);
         T X = p == 0 ? x : (T)0, Y = p == 1 ? x : (T)0;
         a.msg.p[p][e] = X ^ mat_ptr(a, p, 0, 0)[e];
@@ -298,16 +306,17 @@ __device__ __forceinline__ void msb_level_body(const MsbArgs<T> &a, int j, int64
     if (j == 1) {
         and_open(a, e, 0, 0, z);
 #pragma unroll
-        for (int p = 0; p < 2; ++p) { G[p] = z[p]; P[p] = msb_input(a, p, e); }
+        for (int p = 0; p < 2; ++p) { PSML_PARTY_SKIP(a, p) G[p] = z[p]; P[p] = msb_input(a, p, e); }
     } else {
         and_open(a, e, 0, 2 * j - 3, z);
         T zp[2];
         and_open(a, e, 2, 2 * j - 2, zp);
 #pragma unroll
-        for (int p = 0; p < 2; ++p) { G[p] = a.G.p[p][e] ^ z[p]; P[p] = zp[p]; }
+        for (int p = 0; p < 2; ++p) { PSML_PARTY_SKIP(a, p) G[p] = a.G.p[p][e] ^ z[p]; P[p] = zp[p]; }
     }
 #pragma unroll
     for (int p = 0; p < 2; ++p) {
+        PSML_PARTY_SKIP(a, p)
         const int t1 = 2 * j - 1;
         a.msg.p[p][e] = P[p] ^ mat_ptr(a, p, t1, 0)[e];
         a.msg.p[p][a.n + e] = (T)(G[p] << k) ^ mat_ptr(a, p, t1, 1)[e];
@@ -330,6 +339,7 @@ __device__ __forceinline__ void msb_final_body(const MsbArgs<T> &a, const Pair<T
     and_open(a, e, 0, t, z);
 #pragma unroll
     for (int p = 0; p < 2; ++p) {
+        PSML_PARTY_SKIP(a, p)
         T G = a.G.p[p][e] ^ z[p];
         T x = msb_input(a, p, e);
         T b = ((x >> (a.l - 1)) & 1) ^ ((G >> (a.l - 2)) & 1);
@@ -349,6 +359,7 @@ __device__ __forceinline__ void msb_b2a_body(const MsbArgs<T> &a, const Pair<T> 
     const T s = (T)1 - (T)2 * c;
 #pragma unroll
     for (int p = 0; p < 2; ++p) {
+        PSML_PARTY_SKIP(a, p)
         T m = (p == 0 ? c : (T)0) + s * a.mat.p[p][off + a.n + e];
         if (what == 0) {
             msbA.p[p][e] = m;
@@ -364,10 +375,11 @@ __device__ __forceinline__ void msb_b2a_body(const MsbArgs<T> &a, const Pair<T> 
 template <typename T>
 __device__ __forceinline__ void hadamard_open_body(const CPair<T> &mE, const CPair<T> &mF, const CPair<T> &U,
                                                    const CPair<T> &V, const CPair<T> &Z, int trunc,
-                                                   const Pair<T> &C, int64_t i) {
+                                                   const Pair<T> &C, int64_t i, int only = -1) {
     const T e = mE.p[0][i] + mE.p[1][i], f = mF.p[0][i] + mF.p[1][i];
 #pragma unroll
     for (int p = 0; p < 2; ++p) {
+        if (only >= 0 && p != only) continue;
         T c = (T)p * e * f + e * V.p[p][i] + U.p[p][i] * f + Z.p[p][i];
         C.p[p][i] = trunc_share<T>(c, p, trunc);
     }
@@ -377,11 +389,13 @@ __device__ __forceinline__ void hadamard_open_body(const CPair<T> &mE, const CPa
 template <typename T>
 __device__ __forceinline__ void eq9_open_body(const CPair<T> &mE, const CPair<T> &mF, const CPair<T> &U,
                                               const CPair<T> &V, const CPair<T> &Z, int64_t nh, const Pair<T> &y,
-                                              const CPair<T> &Ysub, const Pair<T> &delta, int64_t e) {
+                                              const CPair<T> &Ysub, const Pair<T> &delta, int64_t e,
+                                              int only = -1) {
     const T e1 = mE.p[0][e] + mE.p[1][e], f1 = mF.p[0][e] + mF.p[1][e];
     const T e2 = mE.p[0][e + nh] + mE.p[1][e + nh], f2 = mF.p[0][e + nh] + mF.p[1][e + nh];
 #pragma unroll
     for (int p = 0; p < 2; ++p) {
+        if (only >= 0 && p != only) continue;
         T r1 = (T)p * e1 * f1 + e1 * V.p[p][e] + U.p[p][e] * f1 + Z.p[p][e];
         T r2 = (T)p * e2 * f2 + e2 * V.p[p][e + nh] + U.p[p][e + nh] * f2 + Z.p[p][e + nh];
         T out = r1 - r2;
@@ -411,14 +425,14 @@ __global__ void msb_b2a_kernel(MsbArgs<T> a, Pair<T> msbA, Pair<T> drelu, CPair<
 
 template <typename T>
 __global__ void hadamard_open_kernel(CPair<T> mE, CPair<T> mF, CPair<T> U, CPair<T> V, CPair<T> Z,
-                                     int64_t n, int trunc, Pair<T> C) {
-    PSML_GRID_LOOP(i, n) hadamard_open_body(mE, mF, U, V, Z, trunc, C, i);
+                                     int64_t n, int trunc, Pair<T> C, int only = -1) {
+    PSML_GRID_LOOP(i, n) hadamard_open_body(mE, mF, U, V, Z, trunc, C, i, only);
 }
 
 template <typename T>
 __global__ void eq9_open_kernel(CPair<T> mE, CPair<T> mF, CPair<T> U, CPair<T> V, CPair<T> Z,
-                                int64_t nh, Pair<T> y, CPair<T> Ysub, Pair<T> delta) {
-    PSML_GRID_LOOP(e, nh) eq9_open_body(mE, mF, U, V, Z, nh, y, Ysub, delta, e);
+                                int64_t nh, Pair<T> y, CPair<T> Ysub, Pair<T> delta, int only = -1) {
+    PSML_GRID_LOOP(e, nh) eq9_open_body(mE, mF, U, V, Z, nh, y, Ysub, delta, e, only);
 }
 
 // ---- the whole chain in ONE launch, rounds in order per element ----------------------------------
@@ -613,19 +627,20 @@ __global__ void __launch_bounds__(256) msb_chain_pair_kernel(MsbArgs<T> a, Chain
 // training helpers
 // ---------------------------------------------------------------------------------------------
 template <typename T>
-__global__ void sub_pair_kernel(CPair<T> a, CPair<T> b, int64_t n, Pair<T> c) {
+__global__ void sub_pair_kernel(CPair<T> a, CPair<T> b, int64_t n, Pair<T> c, int only = -1) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-        c.p[0][i] = a.p[0][i] - b.p[0][i];
-        c.p[1][i] = a.p[1][i] - b.p[1][i];
+        if (only != 1) c.p[0][i] = a.p[0][i] - b.p[0][i];
+        if (only != 0) c.p[1][i] = a.p[1][i] - b.p[1][i];
     }
 }
 
 // W^m_i -= trunc_i(g_i, s_grad); W_i = trunc_i(W^m_i, s_fwd)   (R14)
 template <typename T>
-__global__ void update_kernel(Pair<T> Wm, Pair<T> W, CPair<T> g, int64_t n, int s_grad, int s_fwd) {
+__global__ void update_kernel(Pair<T> Wm, Pair<T> W, CPair<T> g, int64_t n, int s_grad, int s_fwd, int only = -1) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
 #pragma unroll
         for (int p = 0; p < 2; ++p) {
+            if (only >= 0 && p != only) continue;
             T wm = Wm.p[p][i] - trunc_share<T>(g.p[p][i], p, s_grad);
             Wm.p[p][i] = wm;
             W.p[p][i] = trunc_share<T>(wm, p, s_fwd);

@@ -781,6 +781,190 @@ static psml_status forward_backward(psml_model_s *m, const T *const X[2], const 
     return backward(m, s);
 }
 
+// ------------------------------------------------------------------------------------------------
+// split deployment: one party per process / GPU (include/psml.h "Split deployment").
+// The same layer sequence as forward()/backward(), but each opening is an exchange through the
+// transport: the party's round kernel writes its masked words to its send buffer, the transport
+// delivers the peer's words into the receive buffer laid out identically, and the next kernel
+// opens send + recv.  The round kernels are the co-resident ones restricted to party `only`
+// (kernels.cuh), so shares and opened values are bit-identical to the co-resident engine.
+// ------------------------------------------------------------------------------------------------
+struct PartyRun {
+    psml_model_s *m;
+    int p;            // this party
+    psml_xport x;
+    cudaStream_t s;
+};
+
+struct Msg {
+    const T *send;
+    T *recv;
+    int64_t words;
+};
+static psml_status xchg(PartyRun &r, std::initializer_list<Msg> msgs) {
+    const void *snd[4];
+    void *rcv[4];
+    int64_t bytes[4];
+    int n = 0;
+    for (const Msg &b : msgs) {
+        snd[n] = b.send; rcv[n] = b.recv; bytes[n] = (int64_t)sizeof(T) * b.words;
+        ++n;
+    }
+    return psml_xport_exchange(r.x, n, snd, rcv, bytes, (psml_stream)r.s);
+}
+
+// one party's pair view: slot p = mine, slot 1 - p = nullptr (never touched by `only` kernels)
+static inline CPair<T> mine_c(int p, const T *v) {
+    CPair<T> c{{nullptr, nullptr}};
+    c.p[p] = v;
+    return c;
+}
+static inline Pair<T> mine(int p, T *v) {
+    Pair<T> c{{nullptr, nullptr}};
+    c.p[p] = v;
+    return c;
+}
+
+// Beaver product (Eqs. 4-8): mask -> exchange E_i, F_i -> open inside the Eq. 8 GEMM.
+static psml_status party_mm(PartyRun &r, const T *A, const T *Bm, int layer, int op, int flags, int trunc, T *C) {
+    psml_model_s *m = r.m;
+    DealItem *it = find_item(m, layer, op, 0);
+    if (!it) return fail(PSML_ERR_STATE, "missing triplet");
+    const int64_t M = it->M, K = it->K, N = it->N;
+    if (2 * (M * K + K * N) > m->ws_words) return fail(PSML_ERR_STATE, "party workspace too small");
+    T *Es = m->ws, *Fs = Es + M * K, *Er = Fs + K * N, *Fr = Er + M * K;
+    psml_ctx ctx = reinterpret_cast<psml_ctx>(m->ctx);
+    const psml_stream ps = (psml_stream)r.s;
+    PSML_TRY(psml_beaver_mask(ctx, r.p, A, Bm, it->U.p[r.p], it->V.p[r.p], M, K, N, flags, Es, Fs, ps));
+    PSML_TRY(xchg(r, {{Es, Er, M * K}, {Fs, Fr, K * N}}));
+    return psml_beaver_open_matmul(ctx, r.p, Es, Er, Fs, Fr, it->U.p[r.p], it->V.p[r.p], it->Z.p[r.p], M, K, N, trunc,
+                                   C, ps);
+}
+
+// MSB chain, one round per kernel with an exchange after each (R9):
+// what 1 = ReLU (y = x . drelu, drelu kept), 2 = Eq. 9 (x = z of n/2; y, delta = y - Ysub).
+static psml_status party_chain(PartyRun &r, const T *x, const DealItem *mat, const DealItem *h, int what, T *y,
+                               T *drelu, const T *Ysub, T *delta) {
+    psml_model_s *m = r.m;
+    const int p = r.p, q = 1 - p;
+    const int64_t n = mat->n;
+    T *ws = m->ws;
+    MsbArgs<T> a;
+    a.x = mine_c(p, x);
+    a.mat = mine_c(p, mat->mat.p[p]);
+    a.G = mine(p, ws + p * n);
+    a.P = mine(p, ws + (2 + p) * n);
+    a.msg = Pair<T>{{ws + 4 * n, ws + 8 * n}};    // msg.p[p]: my send buffer, msg.p[q]: received
+    a.n = n; a.mode = what == 2 ? 1 : 0;
+    a.half = what == 2 ? (T)1 << (m->ctx->ring.frac_bits - 1) : (T)0;
+    a.l = 64; a.L = 6; a.only = p;
+    T *snd = a.msg.p[p], *rcv = a.msg.p[q];
+    const int g = ew_grid(n);
+    {
+        ProfScope prof(PROF_MSB, r.s, 0.0);
+        msb_round0_kernel<T><<<g, EW_THREADS, 0, r.s>>>(a);
+        PSML_LAUNCH_CHECK();
+    }
+    PSML_TRY(xchg(r, {{snd, rcv, 2 * n}}));
+    for (int j = 1; j <= a.L; ++j) {
+        {
+            ProfScope prof(PROF_MSB, r.s, 0.0);
+            msb_level_kernel<T><<<g, EW_THREADS, 0, r.s>>>(a, j);
+            PSML_LAUNCH_CHECK();
+        }
+        PSML_TRY(xchg(r, {{snd, rcv, j < a.L ? 4 * n : 2 * n}}));
+    }
+    Pair<T> none{{nullptr, nullptr}};
+    Pair<T> mE{{a.msg.p[0] + n, a.msg.p[1] + n}}, mF{{a.msg.p[0] + 2 * n, a.msg.p[1] + 2 * n}};
+    const T *U = h->U.p[p], *V = h->V.p[p], *Z = h->Z.p[p];
+    {
+        ProfScope prof(PROF_MSB, r.s, 0.0);
+        msb_final_kernel<T><<<g, EW_THREADS, 0, r.s>>>(a, none);
+        PSML_LAUNCH_CHECK();
+    }
+    PSML_TRY(xchg(r, {{snd, rcv, n}}));   // B2A: c_i = msb_i ^ rB_i
+    {
+        ProfScope prof(PROF_MSB, r.s, 0.0);
+        msb_b2a_kernel<T><<<g, EW_THREADS, 0, r.s>>>(a, none, drelu ? mine(p, drelu) : none, mine_c(p, U), mine_c(p, V),
+                                                     mE, mF, 1);
+        PSML_LAUNCH_CHECK();
+    }
+    PSML_TRY(xchg(r, {{snd + n, rcv + n, 2 * n}}));   // Hadamard x . drelu: E_i, F_i
+    CPair<T> ce{{mE.p[0], mE.p[1]}}, cf{{mF.p[0], mF.p[1]}};
+    ProfScope prof(PROF_HAD, r.s, 0.0);
+    if (what == 1) {
+        hadamard_open_kernel<T><<<g, EW_THREADS, 0, r.s>>>(ce, cf, mine_c(p, U), mine_c(p, V), mine_c(p, Z), n, 0,
+                                                           mine(p, y), p);
+    } else {
+        const int64_t nh = n / 2;
+        eq9_open_kernel<T><<<ew_grid(nh), EW_THREADS, 0, r.s>>>(ce, cf, mine_c(p, U), mine_c(p, V), mine_c(p, Z), nh,
+                                                                mine(p, y), mine_c(p, Ysub),
+                                                                delta ? mine(p, delta) : none, p);
+    }
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
+// Beaver Hadamard c = a (.) b (untruncated), the backprop DReLU product.
+static psml_status party_had(PartyRun &r, const T *a, const T *b, int layer, int slot, T *c) {
+    psml_model_s *m = r.m;
+    DealItem *h = find_item(m, layer, OP_HADAMARD, slot);
+    if (!h) return fail(PSML_ERR_STATE, "missing Hadamard triplet");
+    const int p = r.p, q = 1 - p;
+    const int64_t n = h->n;
+    T *ws = m->ws;
+    Pair<T> mE{{ws, ws + n}}, mF{{ws + 2 * n, ws + 3 * n}};
+    {
+        ProfScope prof(PROF_HAD, r.s, 0.0);
+        hadamard_mask_kernel<T><<<ew_grid(n), EW_THREADS, 0, r.s>>>(mine_c(p, a), mine_c(p, b), mine_c(p, h->U.p[p]),
+                                                                    mine_c(p, h->V.p[p]), n, mE, mF, p);
+        PSML_LAUNCH_CHECK();
+    }
+    PSML_TRY(xchg(r, {{mE.p[p], mE.p[q], n}, {mF.p[p], mF.p[q], n}}));
+    ProfScope prof(PROF_HAD, r.s, 0.0);
+    CPair<T> ce{{mE.p[0], mE.p[1]}}, cf{{mF.p[0], mF.p[1]}};
+    hadamard_open_kernel<T><<<ew_grid(n), EW_THREADS, 0, r.s>>>(ce, cf, mine_c(p, h->U.p[p]), mine_c(p, h->V.p[p]),
+                                                                mine_c(p, h->Z.p[p]), n, 0, mine(p, c), p);
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
+static psml_status party_forward_backward(PartyRun &r, const T *X, const T *Y) {
+    psml_model_s *m = r.m;
+    const int F = m->ctx->ring.frac_bits;
+    const int p = r.p, nl = m->nl;
+    const int64_t B = m->B;
+    m->act[0].p[p] = (T *)X;
+    for (int l = 0; l < nl; ++l) {
+        PSML_TRY(party_mm(r, m->act[l].p[p], m->W[l].p[p], l, OP_FWD, 0, F, m->z[l].p[p]));
+        if (l < nl - 1) {
+            DealItem *mat = find_item(m, l, OP_RELU_MSB, 0), *h = find_item(m, l, OP_HADAMARD, 0);
+            if (!mat || !h) return fail(PSML_ERR_STATE, "missing ReLU material");
+            PSML_TRY(party_chain(r, m->z[l].p[p], mat, h, 1, m->act[l + 1].p[p], m->drelu[l].p[p], nullptr, nullptr));
+        } else if (is_eq9_out(m)) {
+            DealItem *mat = find_item(m, l, OP_EQ9_MSB, 0), *h = find_item(m, l, OP_HADAMARD, 2);
+            if (!mat || !h) return fail(PSML_ERR_STATE, "missing Eq. 9 material");
+            PSML_TRY(party_chain(r, m->z[l].p[p], mat, h, 2, m->yhat.p[p], nullptr, Y, m->delta.p[p]));
+        } else {
+            const int64_t n = B * m->dims[nl];
+            PSML_CUDA_TRY(cudaMemcpyAsync(m->yhat.p[p], m->z[l].p[p], sizeof(T) * n, cudaMemcpyDeviceToDevice, r.s));
+            sub_pair_kernel<T><<<ew_grid(n), EW_THREADS, 0, r.s>>>(mine_c(p, m->z[l].p[p]), mine_c(p, Y), n,
+                                                                    mine(p, m->delta.p[p]), p);
+            PSML_LAUNCH_CHECK();
+        }
+    }
+    T *g[2];
+    for (int l = nl - 1; l >= 0; --l) {
+        gradp(m, l, g);
+        PSML_TRY(party_mm(r, m->act[l].p[p], m->delta.p[p], l, OP_GRADW, PSML_TRANS_A, 0, g[p]));
+        if (l > 0) {
+            PSML_TRY(party_mm(r, m->delta.p[p], m->W[l].p[p], l, OP_GRADIN, PSML_TRANS_B, F, m->tmp.p[p]));
+            PSML_TRY(party_had(r, m->tmp.p[p], m->drelu[l - 1].p[p], l - 1, 1, m->delta.p[p]));
+        }
+    }
+    return PSML_OK;
+}
+
 }  // namespace psml
 
 using namespace psml;
@@ -1164,3 +1348,44 @@ psml_status psml_secure_infer(psml_model m, const void *const X[2], uint32_t ste
     return forward(m, (const T *const *)X, nullptr, (T *const *)Yhat, (cudaStream_t)stream);
 }
 
+
+// ------------------------------------------------------------------------------------------------
+// split deployment ABI
+// ------------------------------------------------------------------------------------------------
+psml_status psml_party_forward_backward(psml_model m, int32_t party, psml_xport x, const void *X_i, const void *Y_i,
+                                        uint32_t step_id, psml_stream stream) {
+    if (!m || !x) return fail(PSML_ERR_INVALID, "null model or transport");
+    if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
+    if (m->d.kind == PSML_CNN) return fail(PSML_ERR_UNSUPPORTED, "split deployment: CNN not built (DESIGN.md §9)");
+    PSML_TRY(check_ptrs({X_i, Y_i}));
+    const int pool = (int)(step_id & 1);
+    if (m->dealt_step[pool] != (int64_t)step_id || !m->dealt_full[pool])
+        return fail(PSML_ERR_STATE, "psml_model_deal(step_id, infer_only=0) must precede the step");
+    m->pool = pool;
+    PartyRun r{m, party, x, (cudaStream_t)stream};
+    PSML_TRY(party_forward_backward(r, (const T *)X_i, (const T *)Y_i));
+    m->grads_ready = true;
+    return PSML_OK;
+}
+
+psml_status psml_party_apply_update(psml_model m, int32_t party, int32_t extra_shift, psml_stream stream) {
+    if (!m) return fail(PSML_ERR_INVALID, "model is null");
+    if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
+    if (extra_shift < 0 || extra_shift > 16) return fail(PSML_ERR_INVALID, "extra_shift out of range");
+    if (!m->grads_ready) return fail(PSML_ERR_STATE, "no gradients: run psml_party_forward_backward first");
+    cudaStream_t s = (cudaStream_t)stream;
+    const int f = m->ctx->ring.frac_bits;
+    const int s_grad = 2 * f + m->d.lr_shift - m->d.master_frac_bits + extra_shift;
+    const int s_fwd = m->d.master_frac_bits - f;
+    for (int l = 0; l < m->nl; ++l) {
+        const int64_t n = m->rows[l] * m->cols[l];
+        T *g[2];
+        gradp(m, l, g);
+        update_kernel<T><<<ew_grid(n), EW_THREADS, 0, s>>>(Pair<T>{{m->Wm[l].p[0], m->Wm[l].p[1]}},
+                                                            Pair<T>{{m->W[l].p[0], m->W[l].p[1]}},
+                                                            CPair<T>{{g[0], g[1]}}, n, s_grad, s_fwd, party);
+        PSML_LAUNCH_CHECK();
+    }
+    m->grads_ready = false;
+    return PSML_OK;
+}

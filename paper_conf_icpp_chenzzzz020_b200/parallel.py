@@ -171,3 +171,61 @@ def split_secure_matmul_compressed(ctx, channel, slot, party, A_i, B_i, U_i, V_i
     Er = channel.exchange((slot, "E"), E)
     Fr = channel.exchange((slot, "F"), F)
     return psml.beaver_open_matmul(ctx, party, E, Er, F, Fr, U_i, V_i, Z_i, M, K, N, trunc)
+
+
+# ---------------------------------------------------------------------------------------------
+# Transports of the split training step (psml_party_forward_backward): every opening round of
+# the step is one symmetric exchange between the two parties of a pair.
+# ---------------------------------------------------------------------------------------------
+def pair_layout(world):
+    """Split deployment over `world` ranks: pair k = (rank k = party 0, rank k + world/2 =
+    party 1).  Returns a function rank -> (party, pair, peer_rank)."""
+    if world < 2 or world % 2:
+        raise ValueError(f"the split deployment needs an even number of ranks, got {world}")
+    half = world // 2
+
+    def of(rank):
+        party, pair = divmod(rank, half)
+        return party, pair, (rank + half) % world
+    return of
+
+
+def host_staged_exchange_fn(peer, group=None):
+    """A psml exchange callback that stages messages through host memory over any
+    torch.distributed backend (gloo): sync the device, D2H, send/recv, H2D, sync."""
+    import torch.distributed as dist
+    from . import psml
+
+    def fn(msgs, _stream):
+        torch.cuda.synchronize()
+        ops, back = [], []
+        for send, recv, nbytes in msgs:
+            if nbytes == 0:
+                continue
+            src = psml.wrap_bytes(send, nbytes).cpu()
+            dst = torch.empty(nbytes, dtype=torch.uint8)
+            ops.append(dist.P2POp(dist.isend, src, peer, group))
+            ops.append(dist.P2POp(dist.irecv, dst, peer, group))
+            back.append((recv, nbytes, dst, src))
+        for req in dist.batch_isend_irecv(ops):
+            req.wait()
+        for recv, nbytes, dst, _ in back:
+            psml.wrap_bytes(recv, nbytes).copy_(dst)
+        torch.cuda.synchronize()
+    return fn
+
+
+def make_transport(party, peer, group=None):
+    """NCCL (library-owned communicator; party 0 creates the unique id and sends it to the peer
+    over the process group) when the backend is nccl, else a host-staged callback."""
+    import torch.distributed as dist
+    from . import psml
+    if dist.get_backend(group) == "nccl":
+        uid = torch.zeros(128, dtype=torch.uint8, device="cuda")
+        if party == 0:
+            uid.copy_(torch.frombuffer(bytearray(psml.nccl_unique_id()), dtype=torch.uint8))
+            dist.send(uid, peer, group)
+        else:
+            dist.recv(uid, peer, group)
+        return psml.Transport.nccl(bytes(uid.cpu().numpy().tobytes()), party)
+    return psml.Transport.callback(host_staged_exchange_fn(peer, group))

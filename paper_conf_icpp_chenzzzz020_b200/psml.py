@@ -15,7 +15,8 @@ LIB_PATH = os.path.join(HERE, "libpsml.so")
 HEADER = os.path.join(os.path.dirname(HERE), "include", "psml.h")
 
 STATUS = {0: "PSML_OK", 1: "PSML_ERR_INVALID", 2: "PSML_ERR_SHAPE", 3: "PSML_ERR_ALIGN",
-          4: "PSML_ERR_UNSUPPORTED", 5: "PSML_ERR_CUDA", 6: "PSML_ERR_NOMEM", 7: "PSML_ERR_STATE"}
+          4: "PSML_ERR_UNSUPPORTED", 5: "PSML_ERR_CUDA", 6: "PSML_ERR_NOMEM", 7: "PSML_ERR_STATE",
+          8: "PSML_ERR_NCCL"}
 TRANS_A, TRANS_B, PAPER_FORM = 1, 2, 4
 LINREG, LOGREG, MLP, CNN = 0, 1, 2, 3
 
@@ -44,6 +45,10 @@ class ModelDesc(ctypes.Structure):
                 ("pair_id", u32), ("cnn_c", i32), ("cnn_h", i32), ("cnn_w", i32), ("cnn_k", i32),
                 ("cnn_cout", i32), ("cnn_hidden", i32), ("cnn_classes", i32)]
 
+
+# psml_exchange_fn (include/psml.h): (user, n, send[], recv[], bytes[], stream) -> 0 on success
+EXCHANGE_FN = ctypes.CFUNCTYPE(i32, vp, i32, ctypes.POINTER(vp), ctypes.POINTER(vp),
+                               ctypes.POINTER(i64), vp)
 
 # name -> (restype, argtypes); mirrors include/psml.h
 _SIGS = {
@@ -90,6 +95,14 @@ _SIGS = {
     "psml_model_capture_step": (i32, [vp, P2, P2, i32, vp]),
     "psml_model_step_graph": (i32, [vp, u32, vp]),
     "psml_model_graph_nodes": (i32, [vp, vp]),
+    "psml_nccl_unique_id": (i32, [vp]),
+    "psml_xport_nccl_create": (i32, [vp, i32, vp]),
+    "psml_xport_callback_create": (i32, [EXCHANGE_FN, vp, vp]),
+    "psml_xport_destroy": (i32, [vp]),
+    "psml_xport_exchange": (i32, [vp, i32, vp, vp, vp, vp]),
+    "psml_xport_stats": (i32, [vp, vp, vp]),
+    "psml_party_forward_backward": (i32, [vp, i32, vp, vp, vp, u32, vp]),
+    "psml_party_apply_update": (i32, [vp, i32, i32, vp]),
 }
 EXPORTS = tuple(_SIGS)
 
@@ -460,6 +473,14 @@ class Model:
     def step_graph(self, step, stream=None):
         _call("psml_model_step_graph", self.handle, step, _stream(stream))
 
+    def party_forward_backward(self, party, xport, X_i, Y_i, step, stream=None):
+        """Split deployment: party `party`'s half of the step, openings through `xport`."""
+        _call("psml_party_forward_backward", self.handle, party, xport.handle, _ptr(X_i), _ptr(Y_i),
+              step, _stream(stream))
+
+    def party_apply_update(self, party, extra_shift=0, stream=None):
+        _call("psml_party_apply_update", self.handle, party, extra_shift, _stream(stream))
+
     def infer(self, X, step, out_shape, stream=None):
         Y = empty_pair(out_shape, self.ctx.l)
         _call("psml_secure_infer", self.handle, _pair(X), step, _pair(Y), _stream(stream))
@@ -475,3 +496,69 @@ class Model:
             self.close()
         except Exception:
             pass
+
+
+# ---------------------------------------------------------------------------------------------
+# split-deployment transports
+# ---------------------------------------------------------------------------------------------
+def nccl_unique_id():
+    buf = (ctypes.c_uint8 * 128)()
+    _call("psml_nccl_unique_id", ctypes.cast(buf, vp))
+    return bytes(buf)
+
+
+class Transport:
+    """psml_xport: how a party's masked messages reach its peer (include/psml.h)."""
+
+    def __init__(self, handle, keep=None):
+        self.handle = handle
+        self._keep = keep   # the ctypes callback must outlive the transport
+
+    @classmethod
+    def nccl(cls, uid, rank):
+        """Library-owned 2-rank NCCL communicator (this party = rank) on the current device."""
+        buf = (ctypes.c_uint8 * 128).from_buffer_copy(uid)
+        h = vp()
+        _call("psml_xport_nccl_create", ctypes.cast(buf, vp), rank, ctypes.byref(h))
+        return cls(h)
+
+    @classmethod
+    def callback(cls, fn):
+        """fn(msgs, stream_ptr): msgs = [(send_ptr, recv_ptr, nbytes)]; must deliver each send
+        buffer to the peer and fill each recv buffer, ordered on the stream."""
+        def tramp(_user, n, send, recv, nbytes, stream):
+            try:
+                fn([(send[k], recv[k], nbytes[k]) for k in range(n)], stream)
+                return 0
+            except Exception as e:   # noqa: BLE001 -- reported through the status code
+                import sys
+                print(f"psml exchange callback failed: {e!r}", file=sys.stderr)
+                return 1
+        cb = EXCHANGE_FN(tramp)
+        h = vp()
+        _call("psml_xport_callback_create", cb, None, ctypes.byref(h))
+        return cls(h, keep=cb)
+
+    def stats(self):
+        b, n = i64(), i64()
+        _call("psml_xport_stats", self.handle, ctypes.byref(b), ctypes.byref(n))
+        return b.value, n.value
+
+    def close(self):
+        if self.handle:
+            lib().psml_xport_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def wrap_bytes(ptr, nbytes):
+    """A uint8 torch tensor aliasing `nbytes` bytes of device memory at `ptr`."""
+    class _Holder:
+        __cuda_array_interface__ = {"shape": (nbytes,), "typestr": "|u1", "data": (ptr, False),
+                                    "version": 3, "strides": None}
+    return torch.as_tensor(_Holder(), device="cuda")

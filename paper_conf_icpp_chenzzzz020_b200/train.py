@@ -146,6 +146,45 @@ class SecureTrainer:
         self.ctx.close()
 
 
+class PartyTrainer(SecureTrainer):
+    """One party of the split deployment (Fig. 1b: the two servers in different
+    processes / GPUs).  The party holds only its own shares; every opening of the step goes
+    through `transport` (psml.Transport: NCCL over NVLink, or a host-staged callback).
+    The dealer runs in each party's process and each party reads only its own half of the
+    material (the offline phase a deployment ships from the client)."""
+
+    def __init__(self, task, W_init, party, transport, batch=128, pair_id=0, **kw):
+        if task == "cnn":
+            raise NotImplementedError("split deployment of the CNN is not built (DESIGN.md §9)")
+        super().__init__(task, W_init, batch=batch, pair_id=pair_id, **kw)
+        self.party = party
+        self.xport = transport
+
+    def share_batch(self, X, Y, step):
+        """Client role: encode + share; this party receives only its own share."""
+        Xs, Ys = super().share_batch(X, Y, step)
+        return Xs[self.party], Ys[self.party]
+
+    def step_party(self, X_i, Y_i, step, dp_group=None, dp_world=1, deal=True):
+        """Forward/backward with per-round exchanges, [all-reduce of this party's gradient
+        share over the party's data-parallel group], update of this party's weights."""
+        if deal:
+            self.model.deal(step)
+        self.model.party_forward_backward(self.party, self.xport, X_i, Y_i, step)
+        if dp_world > 1:
+            ptr, words = self.model.grads()
+            g = _wrap_device_ptr(ptr + 8 * words * self.party, words)
+            ring_allreduce_(g, dp_group)
+        self.model.party_apply_update(self.party, extra_shift=dp_update_shift(dp_world))
+
+    def step(self, X, Y, step):
+        X_i, Y_i = self.share_batch(X, Y, step)
+        self.step_party(X_i, Y_i, step)
+
+    def my_master_share(self, layer):
+        return self.model.get_master(layer)[self.party]
+
+
 def _wrap_device_ptr(ptr, numel, typestr="<i8"):
     """A torch tensor aliasing `numel` 8-byte words of library-owned device memory."""
     class _Holder:

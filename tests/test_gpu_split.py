@@ -111,3 +111,56 @@ def test_split_compressed_transmission(tmp_path):
             assert bool(np.load(tmp_path / f"ok{ep}_{r}.npy")[0]), (r, ep)
         fmts = list(np.load(tmp_path / f"fmt_{r}.npy"))
         assert fmts == ["dense-first", "dense-first", "csr", "dense", "csr", "dense"], fmts
+
+
+# ---------------------------------------------------------------------------------------------
+# Split training step (psml_party_forward_backward): party 0 and party 1 in two processes, every
+# opening (Beaver E/F, each AND round of the MSB chain, the B2A word, the Hadamard E/F) through the
+# library's transport -- here the host-staged gloo callback.  Each party's master-weight share
+# must equal the oracle's simulation of both parties (oracle/protocol.py) after every step.
+# ---------------------------------------------------------------------------------------------
+SPLIT_TASKS = [("linreg", 2), ("logreg", 2), ("mlp", 2)]
+
+
+def _party_train(rank, port, outdir):
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import synth
+    from paper_conf_icpp_chenzzzz020_b200.parallel import make_transport
+    from paper_conf_icpp_chenzzzz020_b200.train import PartyTrainer
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=2)
+    torch.cuda.set_device(0)
+    xp = make_transport(rank, 1 - rank)
+    for task, steps in SPLIT_TASKS:
+        tr = PartyTrainer(task, synth.init_weights(task), rank, xp, backend=1)
+        for s in range(steps):
+            X, Y = synth.batch(task, s)
+            tr.step(torch.from_numpy(X), torch.from_numpy(Y), s)
+            torch.cuda.synchronize()
+            for layer in range(tr.model.n_layers):
+                np.save(os.path.join(outdir, f"{task}_s{s}_l{layer}_{rank}.npy"),
+                        tr.my_master_share(layer).cpu().numpy())
+        tr.close()
+    sent, n_ex = xp.stats()
+    np.save(os.path.join(outdir, f"xstats_{rank}.npy"), np.array([sent, n_ex]))
+    xp.close()
+    dist.destroy_process_group()
+
+
+def test_split_training_matches_oracle(tmp_path):
+    import synth
+    from oracle import protocol as OP
+    mp.spawn(_party_train, args=(_free_port(), str(tmp_path)), nprocs=2, join=True)
+    for task, steps in SPLIT_TASKS:
+        om = OP.Model(task, synth.init_weights(task))
+        for s in range(steps):
+            X, Y = synth.batch(task, s)
+            OP.train_step(om, X, Y, s)
+            for layer in range(len(om.Wm)):
+                for p in range(2):
+                    got = np.load(tmp_path / f"{task}_s{s}_l{layer}_{p}.npy")
+                    assert np.array_equal(got.reshape(om.Wm[layer][p].shape), om.Wm[layer][p]), \
+                        (task, s, layer, p)
+    st = [np.load(tmp_path / f"xstats_{p}.npy") for p in range(2)]
+    assert st[0][1] == st[1][1] > 0 and st[0][0] == st[1][0] > 0   # symmetric exchanges
