@@ -302,7 +302,8 @@ def bench_ours(args):
     # per-kernel-class time inside the same step (CUDA events on the launching stream)
     classes = {}
     base = 3 * (W + K)
-    for cls, name in ((psml.PROF_GEMM, "ring_gemm_cuda_core"), (psml.PROF_MSB, "msb_relu_eq9_rounds"),
+    for cls, name in ((psml.PROF_GEMM, "ring_gemm_cuda_core"), (psml.PROF_TC, "ring_gemm_tcgen05"),
+                      (psml.PROF_MSB, "msb_relu_eq9_rounds"),
                       (psml.PROF_HAD, "hadamard_rounds"), (psml.PROF_DEALER, "dealer"),
                       (psml.PROF_MASK, "beaver_mask")):
         psml.prof_enable(cls)
@@ -425,6 +426,14 @@ def roofline(classes, clocks):
     c = classes[name]
     sec = c["ms_per_launch"] / 1e3
     mp = measured_peaks()
+    if name == "ring_gemm_tcgen05":
+        # tensor (INT8): useful limb-MMA ops = 36 limb pairs x 2 ops per ring MAC
+        peak, src = int8_peak_tops()
+        ach = 36 * 2 * c["work_per_launch"] / sec / 1e12
+        return {"bound": "tensor", "kernel": "tc_seg_kernel (tcgen05 kind::i8, in-kernel limb split)",
+                "achieved": ach, "peak": peak, "unit": "TOPS", "frac": ach / peak, "traffic": None,
+                "peak_source": src,
+                "selection": "largest online-phase kernel class (dealer overlapped)"}
     if name == "ring_gemm_cuda_core":
         # ALU bound: a Z_2^64 multiply-add is 3 IMAD-pipe ops (IMAD.WIDE.U32 + 2 IMAD); B200:
         # 148 SMs x 4 SMSPs x 16 lanes/clk at clocks.max.sm 1965 MHz (B300_MICROARCH rt=2)

@@ -107,6 +107,10 @@ psml_status psml_decode(psml_ring ring, const void *v, int64_t n, double *x, psm
  * x may alias neither x0 nor x1. */
 psml_status psml_share(psml_ring ring, uint64_t seed, uint64_t stream_id, const void *x,
                        int64_t n, void *x0, void *x1, psml_stream stream);
+/* psml_encode then psml_share in one pass: x0 = PRG(seed, "SH", stream_id), x1 = encode(x) - x0.
+ * x: n doubles (device).  Bit-identical to the two calls. */
+psml_status psml_encode_share(psml_ring ring, uint64_t seed, uint64_t stream_id, const double *x,
+                              int64_t n, void *x0, void *x1, psml_stream stream);
 /* x = x0 + x1 mod 2^l (client-side reconstruction). */
 psml_status psml_reconstruct(psml_ring ring, const void *x0, const void *x1, int64_t n, void *x,
                              psml_stream stream);

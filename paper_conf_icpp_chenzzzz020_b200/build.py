@@ -6,7 +6,7 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libpsml.so")
-SOURCES = ["engine.cu", "model.cu", "gemm_tc.cu", "codec.cu", "xport.cu"]
+SOURCES = ["engine.cu", "model.cu", "gemm_tc.cu", "gemm_tcseg.cu", "codec.cu", "xport.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "--expt-relaxed-constexpr", "-Xcompiler", "-fPIC,-fvisibility=hidden", "-Xptxas", "-v"]
@@ -29,7 +29,8 @@ def build(force=False, verbose=False, jobs=4):
     for src in SOURCES:
         obj = os.path.join(CSRC, "build", src.replace(".cu", ".o"))
         os.makedirs(os.path.dirname(obj), exist_ok=True)
-        cmd = [NVCC] + FLAGS + ["-c", os.path.join(CSRC, src), "-o", obj]
+        extra = os.environ.get("PSML_NVCC_EXTRA", "").split()   # e.g. -DTCSEG_TIMING (experiments)
+        cmd = [NVCC] + FLAGS + extra + ["-c", os.path.join(CSRC, src), "-o", obj]
         procs.append((src, subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT)))
         objs.append(obj)
     failed = False

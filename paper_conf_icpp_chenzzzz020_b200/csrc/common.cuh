@@ -63,6 +63,11 @@ struct ProfScope {
     }
 };
 
+// Programmatic dependent launch trigger: lets a dependent kernel launched with
+// cudaLaunchAttributeProgrammaticStreamSerialization start its prologue now (it still waits,
+// with griddepcontrol.wait, for this grid's completion before reading its outputs).
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
 #define PSML_TRY(expr)                          \
     do {                                        \
         psml_status _s = (expr);                \

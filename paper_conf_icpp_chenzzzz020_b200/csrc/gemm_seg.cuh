@@ -236,11 +236,21 @@ __global__ void __launch_bounds__(SegCfg::NT) seg_gemm_kernel(const __grid_const
     cl_finish<T, SegEpi<T>, C>(epi, p, m0, n0, ks, smem, acc);
 }
 
+// tcgen05 form of the same group (gemm_tcseg.cu; l = 64, sm_100, K' <= 16384 per product).
+// PSML_SEG=simt keeps the CUDA-core kernel below.
+bool tc_seg_enabled();
+psml_status tc_seg_group(const SegArgs<uint64_t> *jobs, int njobs, cudaStream_t stream, int sm_count);
+
 // Launch 1..SEG_MAX_JOBS products as one grid; the cluster split ks is chosen for the group.
 template <typename T>
 psml_status launch_seg_group(const SegArgs<T> *jobs, int njobs, cudaStream_t stream, int sm_count) {
     using C = SegCfg;
     if (njobs < 1 || njobs > SEG_MAX_JOBS) return fail(PSML_ERR_INVALID, "seg group: 1..4 jobs");
+    if constexpr (sizeof(T) == 8) {
+        bool ok = tc_seg_enabled();
+        for (int q = 0; q < njobs && ok; ++q) ok = 2 * jobs[q].K <= 16384;
+        if (ok) return tc_seg_group(reinterpret_cast<const SegArgs<uint64_t> *>(jobs), njobs, stream, sm_count);
+    }
     SegGroup<T> g{};
     int64_t tiles = 0, kmax = 0;
     double work = 0;

@@ -40,6 +40,28 @@ __global__ void prg_kernel(PrgKey key, uint64_t offset, int64_t n, T *__restrict
     }
 }
 
+// Client encode + share in one pass: v = encode(x) (R3), x0 = PRG, x1 = v - x0.
+template <typename T>
+__global__ void encode_share_kernel(PrgKey key, int64_t n, int f, const double *__restrict__ x, T *__restrict__ out0,
+                                    T *__restrict__ out1) {
+    constexpr int PB = PerBlock<T>::value;
+    key = live_key(key);
+    const uint64_t last_blk = ((uint64_t)n - 1) / PB;
+    for (uint64_t b = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; b <= last_blk; b += (uint64_t)gridDim.x * blockDim.x) {
+        uint32_t w[16];
+        chacha20_block(key, (uint32_t)b, w);
+#pragma unroll
+        for (int j = 0; j < PB; ++j) {
+            const uint64_t e = b * PB + j;
+            if (e >= (uint64_t)n) continue;
+            const T r = sizeof(T) == 8 ? (T)(((uint64_t)w[2 * j + 1] << 32) | w[2 * j]) : (T)w[j];
+            const T v = (T)(unsigned long long)__double2ll_rn(ldexp(x[e], f));
+            out0[e] = r;
+            out1[e] = v - r;
+        }
+    }
+}
+
 template <typename T>
 __global__ void encode_kernel(const double *__restrict__ x, int64_t n, int f, T *__restrict__ v) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
@@ -515,6 +537,7 @@ __device__ __forceinline__ T peer_of(T v) {
 #define SEL(pair) (p ? (pair).p[1] : (pair).p[0])
 template <typename T, int MODE>
 __global__ void __launch_bounds__(256) msb_chain_pair_kernel(MsbArgs<T> a, ChainOut<T> o) {
+    pdl_trigger();
     constexpr int l = 8 * (int)sizeof(T);
     constexpr int L = sizeof(T) == 8 ? 6 : 5;
     const int lane = threadIdx.x & 31;

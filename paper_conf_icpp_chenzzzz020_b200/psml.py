@@ -65,6 +65,7 @@ _SIGS = {
     "psml_decode": (i32, [Ring, vp, i64, vp, vp]),
     "psml_share": (i32, [Ring, u64, u64, vp, i64, vp, vp, vp]),
     "psml_reconstruct": (i32, [Ring, vp, vp, i64, vp, vp]),
+    "psml_encode_share": (i32, [Ring, u64, u64, vp, i64, vp, vp, vp]),
     "psml_triplet_gen": (i32, [vp, u64, u64, i64, i64, i64, P2, P2, P2, vp]),
     "psml_hadamard_triplet_gen": (i32, [Ring, u64, u64, i64, P2, P2, P2, vp]),
     "psml_msb_material_words": (i64, [Ring, i64]),
@@ -253,6 +254,16 @@ def decode(ring, v, stream=None):
 def share(ring, seed, stream_id, x, out=None, stream=None):
     x0, x1 = out if out is not None else empty_pair(x.shape, ring.l)
     _call("psml_share", ring, seed, stream_id, _ptr(x), x.numel(), _ptr(x0), _ptr(x1),
+          _stream(stream))
+    return x0, x1
+
+
+def encode_share(ring, seed, stream_id, x, out=None, stream=None):
+    """psml_encode + psml_share in one kernel (x: float64 device tensor)."""
+    if x.dtype != torch.float64:
+        raise PsmlError("marshal", 1, "encode_share takes float64")
+    x0, x1 = out if out is not None else empty_pair(x.shape, ring.l)
+    _call("psml_encode_share", ring, seed, stream_id, _ptr(x), x.numel(), _ptr(x0), _ptr(x1),
           _stream(stream))
     return x0, x1
 

@@ -54,10 +54,10 @@ class SecureTrainer:
     # --- client side -----------------------------------------------------------------------
     def share_batch(self, X, Y, step):
         """Encode + share one minibatch on the GPU (X, Y: float64 tensors, host or device)."""
-        x = psml.encode(self.ring, torch.as_tensor(X, dtype=torch.float64))
-        y = psml.encode(self.ring, torch.as_tensor(Y, dtype=torch.float64))
-        Xs = psml.share(self.ring, SHARE_SEED, call_id(self.pair_id, step, 0, OP_SHARE, 0), x)
-        Ys = psml.share(self.ring, SHARE_SEED, call_id(self.pair_id, step, 0, OP_SHARE, 1), y)
+        Xs = psml.encode_share(self.ring, SHARE_SEED, call_id(self.pair_id, step, 0, OP_SHARE, 0),
+                               _dev64(X))
+        Ys = psml.encode_share(self.ring, SHARE_SEED, call_id(self.pair_id, step, 0, OP_SHARE, 1),
+                               _dev64(Y))
         return Xs, Ys
 
     # --- steps --------------------------------------------------------------------------------
@@ -85,10 +85,10 @@ class SecureTrainer:
 
     def graph_step(self, X, Y, step):
         """Client encode + share into the captured buffers, then replay the captured step."""
-        x = psml.encode(self.ring, torch.as_tensor(X, dtype=torch.float64))
-        y = psml.encode(self.ring, torch.as_tensor(Y, dtype=torch.float64))
-        psml.share(self.ring, SHARE_SEED, call_id(self.pair_id, step, 0, OP_SHARE, 0), x, out=self.Xbuf)
-        psml.share(self.ring, SHARE_SEED, call_id(self.pair_id, step, 0, OP_SHARE, 1), y, out=self.Ybuf)
+        psml.encode_share(self.ring, SHARE_SEED, call_id(self.pair_id, step, 0, OP_SHARE, 0), _dev64(X),
+                          out=self.Xbuf)
+        psml.encode_share(self.ring, SHARE_SEED, call_id(self.pair_id, step, 0, OP_SHARE, 1), _dev64(Y),
+                          out=self.Ybuf)
         if self.pipelined and self._next_dealt != step:
             self.model.deal(step)          # prime the pipeline (first step or a jump in step ids)
         self.model.step_graph(step)
@@ -183,6 +183,12 @@ class PartyTrainer(SecureTrainer):
 
     def my_master_share(self, layer):
         return self.model.get_master(layer)[self.party]
+
+
+def _dev64(X):
+    """A contiguous float64 CUDA tensor of the plaintext batch (no copy if it already is one)."""
+    t = torch.as_tensor(X, dtype=torch.float64)
+    return (t if t.is_cuda else t.cuda()).contiguous()
 
 
 def _wrap_device_ptr(ptr, numel, typestr="<i8"):

@@ -61,6 +61,12 @@ def test_encode_decode_share_reconstruct(P, orc, l):
     w0, w1 = orc.share(want, SEED + 1, 42, l)
     assert np.array_equal(to_np(x0), w0) and np.array_equal(to_np(x1), w1)
     assert np.array_equal(to_np(P.reconstruct(ring, x0, x1)), want)
+    # fused client pass (psml_encode_share) == encode then share, on ragged sizes
+    for n in (1, 7, 17, len(x)):
+        xs = torch.from_numpy(x[:n]).cuda()
+        y0, y1 = P.encode_share(ring, SEED + 1, 43, xs)
+        u0, u1 = orc.share(orc.encode(x[:n], l, 13), SEED + 1, 43, l)
+        assert np.array_equal(to_np(y0), u0) and np.array_equal(to_np(y1), u1), n
 
 
 @pytest.mark.parametrize("l", [64, 32])
@@ -99,7 +105,8 @@ def test_hadamard_triplet_and_msb_material(P, orc, ctx):
 
 # --- Beaver matmul -----------------------------------------------------------------------------
 SHAPES = [(4, 4, 4), (3, 5, 2), (128, 784, 1), (784, 128, 1), (128, 784, 128), (128, 128, 10),
-          (784, 128, 128), (100, 37, 65), (257, 129, 200), (64, 3000, 64)]
+          (784, 128, 128), (100, 37, 65), (257, 129, 200), (64, 3000, 64), (130, 8192, 66),
+          (1, 16, 1), (129, 33, 65)]
 
 
 @pytest.mark.parametrize("shape", SHAPES)

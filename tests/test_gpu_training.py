@@ -143,3 +143,20 @@ def test_explicit_mask_round_matches_fused_open():
                         "training_bitexact_vs_oracle or graph_replay", os.path.join(root, "tests", "test_gpu_training.py")],
                        env=env, capture_output=True, text=True, cwd=root)
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
+
+
+def test_cuda_core_seg_gemm_matches_oracle():
+    """PSML_SEG=simt: the opened Beaver products of the training step on the CUDA-core
+    two-segment GEMM instead of the tcgen05 in-kernel-split GEMM (gemm_tcseg.cu, the default);
+    both reproduce the oracle exactly."""
+    import os
+    import subprocess
+    import sys
+    env = dict(os.environ, PSML_SEG="simt")
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu", "-k",
+                        "training_bitexact_vs_oracle or graph_replay or secure_matmul_bitexact",
+                        os.path.join(root, "tests", "test_gpu_training.py"),
+                        os.path.join(root, "tests", "test_gpu_primitives.py")],
+                       env=env, capture_output=True, text=True, cwd=root)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]

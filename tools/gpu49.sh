@@ -1,0 +1,12 @@
+cd $GRAFT_REPO_ROOT
+mkdir -p gpurun_out
+timeout 300 python -m pytest tests/test_gpu_primitives.py -x -q -k "secure_matmul" 2>&1 | tail -2
+timeout 300 python -m pytest tests/test_gpu_training.py -x -q -k "bitexact or graph" 2>&1 | tail -2
+timeout 300 python bench.py --steps 500 --no-cpu-baseline --no-ring-gemm > gpurun_out/b49.json 2> gpurun_out/b49.err
+tail -2 gpurun_out/b49.err
+python -c "
+import json; d=json.load(open('gpurun_out/b49.json'))
+print('value',round(d['value']),'online_graph',round(d.get('online_graph_samples_per_s')),'e2e',round(d['e2e']['value']),'ms',round(d['ms_per_step'],4)); print({k:(round(v['ms_per_step'],4), v['launches_per_step']) for k,v in d['kernel_classes'].items()}); print(d['roofline'])"
+timeout 300 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches49_graph.csv python tools/step_profile.py mlp 4 > gpurun_out/ncu49b.log 2>&1
+timeout 300 ncu --set full --clock-control none --import-source on -k regex:tc_seg -s 12 -c 6 -o gpurun_out/tcseg49 python tools/step_profile.py mlp 3 > gpurun_out/ncu49c.log 2>&1
+tail -1 gpurun_out/ncu49c.log

@@ -1,0 +1,16 @@
+cd $GRAFT_REPO_ROOT
+mkdir -p gpurun_out
+PSML_NVCC_EXTRA=-DTCSEG_TIMING python -m paper_conf_icpp_chenzzzz020_b200.build --force 2>&1 | grep -i error
+stdbuf -o0 -e0 timeout 120 python tools/step_profile.py mlp 3 > gpurun_out/t52.txt 2>&1
+grep tcseg gpurun_out/t52.txt | tail -12
+python -m paper_conf_icpp_chenzzzz020_b200.build --force 2>&1 | grep -i error
+timeout 300 python -m pytest tests/test_gpu_primitives.py -x -q -k "secure_matmul or encode" 2>&1 | tail -2
+timeout 600 python -m pytest tests/test_gpu_training.py tests/test_gpu_split.py -x -q 2>&1 | tail -2
+for pdl in 1; do
+PSML_PDL=$pdl timeout 300 python bench.py --steps 1000 --no-cpu-baseline --no-ring-gemm > gpurun_out/b52.json 2> gpurun_out/b52.err
+tail -2 gpurun_out/b52.err
+python -c "
+import json; d=json.load(open('gpurun_out/b52.json'))
+print('PDL=$pdl value',round(d['value']),'online_graph',round(d.get('online_graph_samples_per_s')),'e2e',round(d['e2e']['value']),'ms',round(d['ms_per_step'],4)); print({k:(round(v['ms_per_step'],4), v['launches_per_step']) for k,v in d['kernel_classes'].items()})"
+done
+timeout 300 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches52_graph.csv python tools/step_profile.py mlp 4 > gpurun_out/ncu52b.log 2>&1
