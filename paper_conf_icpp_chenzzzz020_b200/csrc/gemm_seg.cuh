@@ -174,6 +174,7 @@ __global__ void __launch_bounds__(SegCfg::NT) seg_gemm_kernel(const __grid_const
     const int nch = kend > kbeg ? (int)((kend - kbeg + C::BK - 1) / C::BK) : 0;
     const int tid = threadIdx.x;
     const T *Xp = a.X[p], *Vp = a.V[p];
+    asm volatile("griddepcontrol.wait;" ::: "memory");   // operands come from the predecessor
     auto issue = [&](int c) {
         const int st = c % C::STAGES;
         const int64_t k0 = kbeg + (int64_t)c * C::BK;
@@ -239,6 +240,8 @@ __global__ void __launch_bounds__(SegCfg::NT) seg_gemm_kernel(const __grid_const
 // tcgen05 form of the same group (gemm_tcseg.cu; l = 64, sm_100, K' <= 16384 per product).
 // PSML_SEG=simt keeps the CUDA-core kernel below.
 bool tc_seg_enabled();
+bool tc_seg_forced();   // PSML_SEG=tc: every eligible group on tcgen05 (tests)
+bool pdl_enabled();     // PSML_PDL=0 disables programmatic dependent launch
 psml_status tc_seg_group(const SegArgs<uint64_t> *jobs, int njobs, cudaStream_t stream, int sm_count);
 
 // Launch 1..SEG_MAX_JOBS products as one grid; the cluster split ks is chosen for the group.
@@ -247,9 +250,17 @@ psml_status launch_seg_group(const SegArgs<T> *jobs, int njobs, cudaStream_t str
     using C = SegCfg;
     if (njobs < 1 || njobs > SEG_MAX_JOBS) return fail(PSML_ERR_INVALID, "seg group: 1..4 jobs");
     if constexpr (sizeof(T) == 8) {
+        // tcgen05 once the group has >= 2^25 ring MACs (measured on B200, tools/gpu53-55.sh: the
+        // 128 x 1568 x 128 and 784 x 256 x 128 products of the MLP run 1.4x faster on tcgen05;
+        // the smaller ones are bound by its fixed ~7 us prologue + DSMEM split-K reduction)
         bool ok = tc_seg_enabled();
-        for (int q = 0; q < njobs && ok; ++q) ok = 2 * jobs[q].K <= 16384;
-        if (ok) return tc_seg_group(reinterpret_cast<const SegArgs<uint64_t> *>(jobs), njobs, stream, sm_count);
+        double macs = 0;
+        for (int q = 0; q < njobs && ok; ++q) {
+            ok = 2 * jobs[q].K <= 16384;
+            macs += (double)jobs[q].M * jobs[q].N * 2 * jobs[q].K * jobs[q].nparty;
+        }
+        if (ok && (macs >= (double)(1 << 25) || tc_seg_forced()))
+            return tc_seg_group(reinterpret_cast<const SegArgs<uint64_t> *>(jobs), njobs, stream, sm_count);
     }
     SegGroup<T> g{};
     int64_t tiles = 0, kmax = 0;
@@ -274,11 +285,13 @@ psml_status launch_seg_group(const SegArgs<T> *jobs, int njobs, cudaStream_t str
     cfg.gridDim = dim3((unsigned)tiles, 1, (unsigned)g.ks);
     cfg.blockDim = dim3(C::NT);
     cfg.stream = stream;
-    cudaLaunchAttribute attr[1];
+    cudaLaunchAttribute attr[2];
     attr[0].id = cudaLaunchAttributeClusterDimension;
     attr[0].val.clusterDim.x = 1; attr[0].val.clusterDim.y = 1; attr[0].val.clusterDim.z = (unsigned)g.ks;
+    attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[1].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
     cfg.attrs = attr;
-    cfg.numAttrs = 1;
+    cfg.numAttrs = 2;
     ProfScope prof(PROF_GEMM, stream, work);
     PSML_CUDA_TRY(cudaLaunchKernelEx(&cfg, seg_gemm_kernel<T>, g));
     return PSML_OK;

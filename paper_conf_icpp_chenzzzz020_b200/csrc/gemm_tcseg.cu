@@ -22,12 +22,17 @@
 namespace psml {
 namespace tcseg {
 
-constexpr int BM = 128, BN = 64, BK = 32, NT = 256, STAGES = 3, L = 8;
+constexpr int BM = 128, BN = 64, BK = 32, NT = 256, STAGES = 2, L = 8;
 constexpr int A_TILE = BM * BK;                     // bytes per limb plane of one A block
 constexpr int B_TILE = BN * BK;                     // bytes per limb plane of one B block
-constexpr int STAGE_BYTES = L * (A_TILE + B_TILE);  // 48 KB
+constexpr int STAGE_BYTES = L * (A_TILE + B_TILE);  // 48 KB of limb planes per K block
 constexpr int RED_PITCH = BN + 1;                   // u64 words per row of the reduction tile
-constexpr int PIPE_BYTES = STAGES * STAGE_BYTES;
+// raw uint64 operand words of one K block, landed by cp.async two blocks ahead of their split
+constexpr int RAW_STAGES = 2, RAW_A_PITCH = 34;     // A rows padded to 272 B (16-B aligned)
+constexpr int RAW_A_BYTES = BM * RAW_A_PITCH * 8, RAW_B_BYTES = BK * BN * 8;
+constexpr int RAW_STAGE_BYTES = RAW_A_BYTES + RAW_B_BYTES;
+constexpr int RAW_OFF = STAGES * STAGE_BYTES;
+constexpr int PIPE_BYTES = RAW_OFF + RAW_STAGES * RAW_STAGE_BYTES;
 static_assert(BM * RED_PITCH * 8 <= PIPE_BYTES, "reduction tile must fit the pipeline region");
 constexpr size_t SMEM_BYTES = PIPE_BYTES + 8 * (STAGES + 2) + 16;   // > 114 KB: one CTA per SM
 constexpr int MAX_KS = 16;
@@ -38,6 +43,7 @@ struct Group {
     int tiles_n[SEG_MAX_JOBS], tiles_m[SEG_MAX_JOBS];
     int kb_per_split[SEG_MAX_JOBS];
     int njobs, ks;
+    int debug_mmas;   // TCSEG_TIMING builds: issue only limb pairs with 8 p + q < debug_mmas
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -118,6 +124,16 @@ __device__ __forceinline__ void limbs4(const uint64_t *v, uint32_t out[8]) {
 }
 
 __device__ __forceinline__ uint64_t ldg(const uint64_t *p) { return __ldg((const unsigned long long *)p); }
+__device__ __forceinline__ void cp_async16(void *dst, const void *src, bool ok) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_u32(dst)), "l"(src), "r"(ok ? 16 : 0)
+                 : "memory");
+}
+__device__ __forceinline__ void cp_async8(void *dst, const void *src, bool ok) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;" ::"r"(smem_u32(dst)), "l"(src), "r"(ok ? 8 : 0)
+                 : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait1() { asm volatile("cp.async.wait_group 1;" ::: "memory"); }
 
 constexpr int ZPF = 8;   // epilogue Z words prefetched per thread (ks >= 4)
 
@@ -206,55 +222,82 @@ __global__ void __launch_bounds__(NT, 1) tc_seg_kernel(const __grid_constant__ G
         }
     }
 
-    // load assignment: A unit = (row ar, 16-k half ac); B unit = (column bn, 8-k quarter bq)
+    // stash assignment: A unit = (row ar, 16-k half ac); B unit = (column bn, 8-k quarter bq)
     const int ar = tid >> 1, ac = tid & 1;
     const int bn = tid & 63, bq = tid >> 6;
-    const int64_t arow = m0 + ar, bcol = n0 + bn;
-    const bool arow_ok = arow < M, bcol_ok = bcol < N;
-    const int64_t arow_c = arow_ok ? arow : M - 1, bcol_c = bcol_ok ? bcol : N - 1;
-    const bool a_vec = (K % 16) == 0;   // a 16-word run never straddles the X | E boundary
-    uint64_t ra[16], rb[8];
-    auto load = [&](int kb) {
-        const int64_t ka = (int64_t)kb * BK + 16 * ac;
-        if (a_vec && arow_ok && ka + 16 <= Kext) {
-            const uint64_t *src = ka < K ? Xp + arow * K + ka : Ep + arow * K + (ka - K);
+    // cp.async of one K block's raw words into raw stage rs (zero-filled outside the operands):
+    // 16-byte chunks when the X | E boundary and row starts allow it (K, N even), else 8-byte
+    auto al16 = [](const void *q) { return ((uintptr_t)q & 15) == 0; };
+    const bool a16 = (K % 2) == 0 && al16(Xp) && al16(Ep), b16 = (N % 2) == 0 && al16(Fp) && al16(Vp);
+    auto issue = [&](int kb, int rs) {
+        uint8_t *ra = smem + RAW_OFF + rs * RAW_STAGE_BYTES, *rb = ra + RAW_A_BYTES;
+        const int64_t k0 = (int64_t)kb * BK;
+        if (a16) {
 #pragma unroll
-            for (int j = 0; j < 16; j += 2) {
-                const ulonglong2 v = __ldg((const ulonglong2 *)(src + j));
-                ra[j] = v.x;
-                ra[j + 1] = v.y;
+            for (int u = 0; u < BM * BK / 2 / NT; ++u) {
+                const int c = tid + NT * u, row = c >> 4, kk = (c & 15) * 2;
+                const int64_t m = m0 + row, k = k0 + kk;
+                const bool ok = m < M && k < Kext;
+                const int64_t mc = ok ? m : 0, kc = ok ? k : 0;
+                const uint64_t *src = kc < K ? Xp + mc * K + kc : Ep + mc * K + (kc - K);
+                cp_async16(ra + row * RAW_A_PITCH * 8 + kk * 8, src, ok);
             }
         } else {
-#pragma unroll
-            for (int j = 0; j < 16; ++j) {
-                const int64_t k = ka + j;
-                const int64_t kc = k < Kext ? k : Kext - 1;
-                const uint64_t v = kc < K ? ldg(Xp + arow_c * K + kc) : ldg(Ep + arow_c * K + (kc - K));
-                ra[j] = (arow_ok && k < Kext) ? v : 0ull;
+#pragma unroll 4
+            for (int u = 0; u < BM * BK / NT; ++u) {
+                const int c = tid + NT * u, row = c >> 5, kk = c & 31;
+                const int64_t m = m0 + row, k = k0 + kk;
+                const bool ok = m < M && k < Kext;
+                const int64_t mc = ok ? m : 0, kc = ok ? k : 0;
+                const uint64_t *src = kc < K ? Xp + mc * K + kc : Ep + mc * K + (kc - K);
+                cp_async8(ra + row * RAW_A_PITCH * 8 + kk * 8, src, ok);
             }
         }
-        const int64_t kb8 = (int64_t)kb * BK + 8 * bq;
+        if (b16) {
 #pragma unroll
-        for (int j = 0; j < 8; ++j) {
-            const int64_t k = kb8 + j;
-            const int64_t kc = k < Kext ? k : Kext - 1;
-            const uint64_t v = kc < K ? ldg(Fp + kc * N + bcol_c) : ldg(Vp + (kc - K) * N + bcol_c);
-            rb[j] = (bcol_ok && k < Kext) ? v : 0ull;
+            for (int u = 0; u < BK * BN / 2 / NT; ++u) {
+                const int c = tid + NT * u, kk = c >> 5, nn = (c & 31) * 2;
+                const int64_t k = k0 + kk, n = n0 + nn;
+                const bool ok = k < Kext && n < N;
+                const int64_t kc = ok ? k : 0, ncl = ok ? n : 0;
+                const uint64_t *src = kc < K ? Fp + kc * N + ncl : Vp + (kc - K) * N + ncl;
+                cp_async16(rb + (kk * BN + nn) * 8, src, ok);
+            }
+        } else {
+#pragma unroll 4
+            for (int u = 0; u < BK * BN / NT; ++u) {
+                const int c = tid + NT * u, kk = c >> 6, nn = c & 63;
+                const int64_t k = k0 + kk, n = n0 + nn;
+                const bool ok = k < Kext && n < N;
+                const int64_t kc = ok ? k : 0, ncl = ok ? n : 0;
+                const uint64_t *src = kc < K ? Fp + kc * N + ncl : Vp + (kc - K) * N + ncl;
+                cp_async8(rb + (kk * BN + nn) * 8, src, ok);
+            }
         }
     };
     const int a_off = (((ar >> 3) * 2 + ac) * 128) + (ar & 7) * 16;
     const int b_off = (((bn >> 3) * 2 + (bq >> 1)) * 128) + (bn & 7) * 16 + (bq & 1) * 8;
-    auto stash = [&](int st) {
+    auto stash = [&](int rs, int st) {
+        const uint8_t *ra = smem + RAW_OFF + rs * RAW_STAGE_BYTES, *rb = ra + RAW_A_BYTES;
         uint8_t *sa = smem + st * STAGE_BYTES, *sb = sa + L * A_TILE;
+        uint64_t va[16], vb[8];
+#pragma unroll
+        for (int j = 0; j < 16; j += 2) {
+            const ulonglong2 v = *(const ulonglong2 *)(ra + ar * RAW_A_PITCH * 8 + (16 * ac + j) * 8);
+            va[j] = v.x;
+            va[j + 1] = v.y;
+        }
+#pragma unroll
+        for (int j = 0; j < 8; ++j) vb[j] = *(const uint64_t *)(rb + ((8 * bq + j) * BN + bn) * 8);
         uint32_t w[4][8];
 #pragma unroll
-        for (int q = 0; q < 4; ++q) limbs4(ra + 4 * q, w[q]);
+        for (int q = 0; q < 4; ++q) limbs4(va + 4 * q, w[q]);
 #pragma unroll
         for (int l = 0; l < L; ++l)
             *(uint4 *)(sa + l * A_TILE + a_off) = make_uint4(w[0][l], w[1][l], w[2][l], w[3][l]);
         uint32_t u[2][8];
-        limbs4(rb, u[0]);
-        limbs4(rb + 4, u[1]);
+        limbs4(vb, u[0]);
+        limbs4(vb + 4, u[1]);
 #pragma unroll
         for (int l = 0; l < L; ++l) *(uint2 *)(sb + l * B_TILE + b_off) = make_uint2(u[0][l], u[1][l]);
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // generic writes -> tensor core
@@ -264,14 +307,37 @@ __global__ void __launch_bounds__(NT, 1) tc_seg_kernel(const __grid_constant__ G
     // output, complete before the predecessor kernel started) overlapped the predecessor; the
     // operands X_p / E / F it produces are read only after this wait.
     asm volatile("griddepcontrol.wait;" ::: "memory");
-    if (nblk > 0) load(kb0);
+    if (nblk > 0) issue(kb0, 0);
+    cp_async_commit();
+    if (nblk > 1) issue(kb0 + 1, 1);
+    cp_async_commit();
     TS(2);
     for (int i = 0; i < nblk; ++i) {
-        const int st = i % STAGES;
+        const int st = i % STAGES, rs = i % RAW_STAGES;
+#ifdef TCSEG_TIMING
+        uint64_t tq0, tq1, tq2, tq3, tq4;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tq0));
+#endif
+        cp_async_wait1();   // this thread's chunks of block i have landed
+        __syncthreads();    // ... and every thread's
+#ifdef TCSEG_TIMING
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tq1));
+#endif
         if (i >= STAGES) mbar_wait(smem_u32(&empty[st]), (uint32_t)((i / STAGES - 1) & 1));
-        stash(st);
-        if (i + 1 < nblk) load(kb0 + i + 1);   // next block's words in flight during the MMAs
-        __syncthreads();
+#ifdef TCSEG_TIMING
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tq2));
+#endif
+        stash(rs, st);
+#ifdef TCSEG_TIMING
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tq3));
+#endif
+        __syncthreads();    // limb stage st complete; raw stage rs free
+#ifdef TCSEG_TIMING
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tq4));
+        if (tid == 0 && blockIdx.x == 0 && blockIdx.z == 0 && gridDim.x == 4)
+            printf("  blk i=%d: wait_data %llu wait_empty %llu stash %llu sync %llu\n", i, tq1 - tq0, tq2 - tq1,
+                   tq3 - tq2, tq4 - tq3);
+#endif
         if (tid == 0) {
             fence_after();
             const uint32_t sa = smem_u32(smem + st * STAGE_BYTES), sb = sa + L * A_TILE;
@@ -279,12 +345,18 @@ __global__ void __launch_bounds__(NT, 1) tc_seg_kernel(const __grid_constant__ G
             for (int pa = 0; pa < L; ++pa) {
                 const uint64_t ad = sdesc(sa + pa * A_TILE);
 #pragma unroll
-                for (int qb = 0; qb < L - pa; ++qb)
+                for (int qb = 0; qb < L - pa; ++qb) {
+#ifdef TCSEG_TIMING
+                    if (g.debug_mmas && pa * 8 + qb >= g.debug_mmas) continue;   // timing experiments only
+#endif
                     mma_i8(tmem + (uint32_t)((pa + qb) * BN), ad, sdesc(sb + qb * B_TILE), IDESC,
                            (i > 0 || pa > 0) ? 1u : 0u);
+                }
             }
             commit(smem_u32(&empty[st]));
         }
+        if (i + 2 < nblk) issue(kb0 + i + 2, rs);
+        cp_async_commit();
     }
     if (tid == 0) commit(smem_u32(accum));
     TS(3);
@@ -370,6 +442,15 @@ __global__ void __launch_bounds__(NT, 1) tc_seg_kernel(const __grid_constant__ G
 
 }  // namespace tcseg
 
+bool tc_seg_forced() {
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("PSML_SEG");
+        v = (e && e[0] == 't') ? 1 : 0;
+    }
+    return v == 1;
+}
+
 bool tc_seg_enabled() {
     static int v = -1;
     if (v < 0) {
@@ -385,8 +466,8 @@ bool tc_seg_enabled() {
     return v == 1;
 }
 
-// PSML_PDL=0 disables programmatic dependent launch of the GEMM after its producer kernel.
-static bool pdl_enabled() {
+// PSML_PDL=0 disables programmatic dependent launch of the GEMMs after their producer kernels.
+bool pdl_enabled() {
     static int v = -1;
     if (v < 0) {
         const char *e = getenv("PSML_PDL");
@@ -435,6 +516,9 @@ psml_status tc_seg_group(const SegArgs<uint64_t> *jobs, int njobs, cudaStream_t 
     }
     g.tile_begin[njobs] = tiles;
     g.njobs = njobs;
+#ifdef TCSEG_TIMING
+    if (const char *e = getenv("PSML_TCSEG_MMAS")) g.debug_mmas = atoi(e);
+#endif
     int ks = 1;
     while (ks < max_ks && tiles * ks * 2 <= sm_count && nkb_max >= ks * 2) ks *= 2;
     g.ks = ks;

@@ -145,14 +145,16 @@ def test_explicit_mask_round_matches_fused_open():
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
 
 
-def test_cuda_core_seg_gemm_matches_oracle():
-    """PSML_SEG=simt: the opened Beaver products of the training step on the CUDA-core
-    two-segment GEMM instead of the tcgen05 in-kernel-split GEMM (gemm_tcseg.cu, the default);
-    both reproduce the oracle exactly."""
+@pytest.mark.parametrize("mode", ["simt", "tc"])
+def test_seg_gemm_backends_match_oracle(mode):
+    """PSML_SEG=simt: every opened Beaver product of the training step on the CUDA-core
+    two-segment GEMM; PSML_SEG=tc: every eligible one on the tcgen05 in-kernel-split GEMM
+    (gemm_tcseg.cu; by default only groups of >= 2^25 ring MACs go there).  Both reproduce the
+    oracle exactly."""
     import os
     import subprocess
     import sys
-    env = dict(os.environ, PSML_SEG="simt")
+    env = dict(os.environ, PSML_SEG=mode)
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
     r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu", "-k",
                         "training_bitexact_vs_oracle or graph_replay or secure_matmul_bitexact",
