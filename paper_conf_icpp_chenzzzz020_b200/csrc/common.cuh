@@ -67,6 +67,26 @@ struct ProfScope {
 // cudaLaunchAttributeProgrammaticStreamSerialization start its prologue now (it still waits,
 // with griddepcontrol.wait, for this grid's completion before reading its outputs).
 __device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+// Wait for the predecessor grid's completion and memory flush (a no-op without a programmatic
+// dependency).  Every PDL-launched kernel calls it before touching its predecessor's outputs.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+bool pdl_enabled();   // PSML_PDL=0 disables programmatic dependent launch
+
+// <<<grid, block, 0, s>>> with programmatic stream serialization (PDL): the kernel may be
+// scheduled while its predecessor drains; it must pdl_wait() before reading the predecessor's data.
+template <typename... KArgs, typename... Args>
+cudaError_t launch_pdl(void (*k)(KArgs...), dim3 grid, dim3 block, cudaStream_t s, Args... args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, k, args...);
+}
 
 #define PSML_TRY(expr)                          \
     do {                                        \

@@ -44,6 +44,7 @@ struct OpenList {
 template <typename T>
 __global__ void __launch_bounds__(256) open_list_kernel(const __grid_constant__ OpenList<T> L) {
     pdl_trigger();
+    pdl_wait();
     __shared__ T tile[2][32][33];
     const int64_t t = blockIdx.x;
     int q = 0;
@@ -114,6 +115,7 @@ struct HadFused {
 template <typename T>
 __global__ void __launch_bounds__(256) had_fused_kernel(const __grid_constant__ HadFused<T> h) {
     pdl_trigger();
+    pdl_wait();
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < h.n; i += (int64_t)gridDim.x * blockDim.x) {
         const T u0 = h.U[0][i], u1 = h.U[1][i], v0 = h.V[0][i], v1 = h.V[1][i];
         const T E = (T)(h.a[0][i] - u0) + (T)(h.a[1][i] - u1);
@@ -137,6 +139,7 @@ struct DeltaFused {
 template <typename T>
 __global__ void __launch_bounds__(256) delta_fused_kernel(const __grid_constant__ DeltaFused<T> d) {
     pdl_trigger();
+    pdl_wait();
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < d.n; i += (int64_t)gridDim.x * blockDim.x) {
         const T z0 = d.z[0][i], z1 = d.z[1][i];
         const T d0 = z0 - d.Y[0][i], d1 = z1 - d.Y[1][i];
@@ -160,6 +163,8 @@ struct UpdateAll {
 
 template <typename T>
 __global__ void __launch_bounds__(256) update_all_kernel(const __grid_constant__ UpdateAll<T> u) {
+    pdl_trigger();
+    pdl_wait();
     const int64_t total = u.begin[u.nl];
     for (int64_t x = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; x < total; x += (int64_t)gridDim.x * blockDim.x) {
         int l = 0;

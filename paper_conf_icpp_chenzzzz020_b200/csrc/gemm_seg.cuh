@@ -174,7 +174,8 @@ __global__ void __launch_bounds__(SegCfg::NT) seg_gemm_kernel(const __grid_const
     const int nch = kend > kbeg ? (int)((kend - kbeg + C::BK - 1) / C::BK) : 0;
     const int tid = threadIdx.x;
     const T *Xp = a.X[p], *Vp = a.V[p];
-    asm volatile("griddepcontrol.wait;" ::: "memory");   // operands come from the predecessor
+    pdl_trigger();
+    pdl_wait();   // operands come from the predecessor
     auto issue = [&](int c) {
         const int st = c % C::STAGES;
         const int64_t k0 = kbeg + (int64_t)c * C::BK;

@@ -306,7 +306,8 @@ __global__ void __launch_bounds__(NT, 1) tc_seg_kernel(const __grid_constant__ G
     // Programmatic dependent launch: everything above (barriers, TMEM, Z prefetch -- the dealer's
     // output, complete before the predecessor kernel started) overlapped the predecessor; the
     // operands X_p / E / F it produces are read only after this wait.
-    asm volatile("griddepcontrol.wait;" ::: "memory");
+    pdl_trigger();
+    pdl_wait();
     if (nblk > 0) issue(kb0, 0);
     cp_async_commit();
     if (nblk > 1) issue(kb0 + 1, 1);

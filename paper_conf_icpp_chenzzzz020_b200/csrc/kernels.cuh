@@ -538,6 +538,7 @@ __device__ __forceinline__ T peer_of(T v) {
 template <typename T, int MODE>
 __global__ void __launch_bounds__(256) msb_chain_pair_kernel(MsbArgs<T> a, ChainOut<T> o) {
     pdl_trigger();
+    pdl_wait();
     constexpr int l = 8 * (int)sizeof(T);
     constexpr int L = sizeof(T) == 8 ? 6 : 5;
     const int lane = threadIdx.x & 31;

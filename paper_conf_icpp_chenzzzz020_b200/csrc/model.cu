@@ -704,7 +704,7 @@ static psml_status fused_forward_backward(psml_model_s *m, const T *const X[2], 
         L.n = n;
         L.tile_begin[n] = tiles;
         ProfScope prof(PROF_MASK, s, 0.0);
-        open_list_kernel<T><<<(unsigned)tiles, dim3(32, 8), 0, s>>>(L);
+        PSML_CUDA_TRY(launch_pdl(open_list_kernel<T>, dim3((unsigned)tiles), dim3(32, 8), s, L));
         PSML_LAUNCH_CHECK();
     }
     // 2. forward
@@ -741,7 +741,7 @@ static psml_status fused_forward_backward(psml_model_s *m, const T *const X[2], 
                 }
                 d.n = B * w;
                 d.em = em;
-                delta_fused_kernel<T><<<ew_grid(d.n), EW_THREADS, 0, s>>>(d);
+                PSML_CUDA_TRY(launch_pdl(delta_fused_kernel<T>, dim3(ew_grid(d.n)), dim3(EW_THREADS), s, d));
                 PSML_LAUNCH_CHECK();
             }
         }
@@ -768,7 +768,7 @@ static psml_status fused_forward_backward(psml_model_s *m, const T *const X[2], 
             hf.em.n = 1;
             if (l - 1 > 0) { hf.em.e[1] = emitA(l - 1, OP_GRADIN, B, w, 0); hf.em.n = 2; }
             ProfScope prof(PROF_HAD, s, 0.0);
-            had_fused_kernel<T><<<ew_grid(hf.n), EW_THREADS, 0, s>>>(hf);
+            PSML_CUDA_TRY(launch_pdl(had_fused_kernel<T>, dim3(ew_grid(hf.n)), dim3(EW_THREADS), s, hf));
             PSML_LAUNCH_CHECK();
         }
     }
@@ -1194,7 +1194,7 @@ psml_status psml_train_apply_update(psml_model m, int32_t extra_shift, psml_stre
         }
         u.begin[m->nl] = tot;
         u.nl = m->nl; u.s_grad = s_grad; u.s_fwd = s_fwd;
-        update_all_kernel<T><<<ew_grid(tot), EW_THREADS, 0, s>>>(u);
+        PSML_CUDA_TRY(launch_pdl(update_all_kernel<T>, dim3(ew_grid(tot)), dim3(EW_THREADS), s, u));
         PSML_LAUNCH_CHECK();
         m->grads_ready = false;
         return PSML_OK;

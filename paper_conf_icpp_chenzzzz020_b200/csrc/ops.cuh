@@ -236,9 +236,11 @@ psml_status msb_chain(const T *const x[2], int64_t n, const T *const mat[2], int
     if (chain_mode() == 0) {   // one launch; lane pair = (party 0, party 1) of one element
         const int64_t threads = what == 2 ? ((n / 2 + 7) / 8) * 32 : 2 * n;
         const int blocks = (int)((threads + EW_THREADS - 1) / EW_THREADS);
-        if (what == 0) msb_chain_pair_kernel<T, 0><<<blocks, EW_THREADS, 0, s>>>(a, o);
-        else if (what == 1) msb_chain_pair_kernel<T, 1><<<blocks, EW_THREADS, 0, s>>>(a, o);
-        else msb_chain_pair_kernel<T, 2><<<blocks, EW_THREADS, 0, s>>>(a, o);
+        cudaError_t e;
+        if (what == 0) e = launch_pdl(msb_chain_pair_kernel<T, 0>, dim3(blocks), dim3(EW_THREADS), s, a, o);
+        else if (what == 1) e = launch_pdl(msb_chain_pair_kernel<T, 1>, dim3(blocks), dim3(EW_THREADS), s, a, o);
+        else e = launch_pdl(msb_chain_pair_kernel<T, 2>, dim3(blocks), dim3(EW_THREADS), s, a, o);
+        if (e != cudaSuccess) return fail(PSML_ERR_CUDA, std::string("msb chain launch: ") + cudaGetErrorString(e));
         PSML_LAUNCH_CHECK();
         return PSML_OK;
     }
