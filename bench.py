@@ -277,6 +277,13 @@ def bench_ours(args):
         out_host[1].view(-1).copy_(y1, non_blocking=True)
     t_e2e = max_over_ranks(timed(e2e_step, K, 2 * (W + K)), world)
 
+    # secure inference (the forward half): client share + inference dealer + forward
+    def infer_step(s):
+        i = s % nb
+        Xsh, _ = tr.share_batch(Xs[i], Ys[i], s)
+        tr.infer_shares(Xsh, s)
+    t_inf = max_over_ranks(timed(infer_step, K, 10 * (W + K)), world)
+
     samples = BATCH * K * world
     result = {
         "metric": METRIC, "value": samples / t_dev, "unit": "samples/s", "n_gpus": world,
@@ -291,6 +298,7 @@ def bench_ours(args):
         "online_samples_per_s": samples / t_on,
         "online_graph_samples_per_s": (samples / t_on_graph) if t_on_graph else None,
         "eager_samples_per_s": samples / t_eager,
+        "infer_samples_per_s": samples / t_inf,
         "cuda_graph": {"kernel_nodes_per_step": n_nodes,
                        "note": "value/e2e replay one captured graph per step (dealer + online "
                                "step + update); online/eager figures use per-kernel launches"},
@@ -418,9 +426,27 @@ def measured_peaks():
         return {}
 
 
+def committed_traffic(name):
+    """DRAM bytes per launch of kernel class `name` from the committed ncu --set full capture
+    (profiles/r01c_traffic.json), or None."""
+    try:
+        t = json.load(open(os.path.join(ROOT, "profiles", "r01c_traffic.json")))
+        return t[name]["bytes_per_launch_avg"], t["source"]
+    except (OSError, ValueError, KeyError):
+        return None, None
+
+
 def roofline(classes, clocks):
     """Roofline of the dominant kernel class: the largest ONLINE-phase class of the step (the
     dealer runs concurrently with the online phase in the pipelined graph), DESIGN.md Sec. 8."""
+    r = _roofline(classes, clocks)
+    r["traffic"], src = committed_traffic(r["class"])
+    if src:
+        r["traffic_unit"], r["traffic_source"] = "bytes per launch", src
+    return r
+
+
+def _roofline(classes, clocks):
     online = [k for k in classes if k != "dealer"]
     name = max(online, key=lambda k: classes[k]["ms_per_step"])
     c = classes[name]
@@ -430,7 +456,7 @@ def roofline(classes, clocks):
         # tensor (INT8): useful limb-MMA ops = 36 limb pairs x 2 ops per ring MAC
         peak, src = int8_peak_tops()
         ach = 36 * 2 * c["work_per_launch"] / sec / 1e12
-        return {"bound": "tensor", "kernel": "tc_seg_kernel (tcgen05 kind::i8, in-kernel limb split)",
+        return {"bound": "tensor", "class": name, "kernel": "tc_seg_kernel (tcgen05 kind::i8, in-kernel limb split)",
                 "achieved": ach, "peak": peak, "unit": "TOPS", "frac": ach / peak, "traffic": None,
                 "peak_source": src,
                 "selection": "largest online-phase kernel class (dealer overlapped)"}
@@ -439,13 +465,14 @@ def roofline(classes, clocks):
         # 148 SMs x 4 SMSPs x 16 lanes/clk at clocks.max.sm 1965 MHz (B300_MICROARCH rt=2)
         peak = 148 * 64 / 3 * 1.965e9 / 1e12
         ach = c["work_per_launch"] / sec / 1e12
-        return {"bound": "alu", "kernel": name, "achieved": ach, "peak": peak,
+        return {"bound": "alu", "class": name, "kernel": "seg_gemm_kernel (CUDA-core two-segment Beaver GEMM)",
+                "achieved": ach, "peak": peak,
                 "unit": "T ring-MAC/s", "frac": ach / peak, "traffic": None,
                 "peak_source": "derived: 148 SM x 64 IMAD/clk / 3 IMAD per u64 MAC x 1965 MHz",
                 "selection": "largest online-phase kernel class (dealer overlapped)"}
     peak = mp.get("hbm_gbs", 6650.0)
     ach = c["work_per_launch"] / sec / 1e9
-    return {"bound": "hbm", "kernel": name, "achieved": ach, "peak": peak, "unit": "GB/s",
+    return {"bound": "hbm", "class": name, "kernel": name, "achieved": ach, "peak": peak, "unit": "GB/s",
             "frac": ach / peak, "traffic": None,
             "peak_source": "measured" if "hbm_gbs" in mp else "fallback",
             "selection": "largest online-phase kernel class (dealer overlapped)"}
@@ -491,6 +518,49 @@ def ring_gemm_figure(n=4096, l=64, reps=5):
                          "achieved": tops, "peak": peak, "unit": "TOPS", "frac": tops / peak,
                          "traffic": None, "peak_source": src},
             "ring_tmacs": n ** 3 / (ms / 1e3) / 1e12}
+
+
+def beaver_latency_figure(reps=2000):
+    """BASELINE config 1: one Beaver secure matmul A 128x784 . B 784x1 in Z_2^64 (both parties
+    co-resident, one linear-regression minibatch), per-call device latency p50/p99 over `reps`
+    calls (CUDA events around each call), beside the oracle's per-call time on the same inputs."""
+    import numpy as np
+    import torch
+    from paper_conf_icpp_chenzzzz020_b200 import psml
+    M, K, N = 128, 784, 1
+    ctx = psml.Ctx(l=64)
+    ring = ctx.ring
+    A = psml.share(ring, 7, 1, psml.prg_fill(ring, 1, psml.tag("cA"), 0, M * K).view(M, K))
+    B = psml.share(ring, 7, 2, psml.prg_fill(ring, 1, psml.tag("cB"), 0, K * N).view(K, N))
+    U, V, Z = psml.triplet_gen(ctx, 3, 0, M, K, N)
+    C = psml.empty_pair((M, N), 64)
+    for _ in range(20):
+        psml.secure_matmul(ctx, A, B, U, V, Z, M, K, N, trunc=13, out=C)
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(reps)]
+    torch.cuda.synchronize()
+    for a, b in evs:
+        a.record()
+        psml.secure_matmul(ctx, A, B, U, V, Z, M, K, N, trunc=13, out=C)
+        b.record()
+    torch.cuda.synchronize()
+    us = np.array([a.elapsed_time(b) * 1e3 for a, b in evs])
+    # the oracle on the same shares and triplet
+    from oracle import core as orc
+    host = lambda t: t.cpu().numpy()  # noqa: E731
+    An, Bn = [host(t) for t in A], [host(t) for t in B]
+    trip = [host(t) for t in (U[0], U[1], V[0], V[1], Z[0], Z[1])]
+    t0 = time.perf_counter()
+    n_or = 0
+    while time.perf_counter() - t0 < 1.0:
+        want = orc.beaver_matmul(An, Bn, trip, trunc=13)
+        n_or += 1
+    t_or = (time.perf_counter() - t0) / n_or * 1e6
+    ok = all(np.array_equal(host(C[i]), want[i]) for i in range(2))
+    ctx.close()
+    return {"config": "single Beaver secure matmul, 2 parties co-resident, Z_2^64, A 128x784 . B 784x1",
+            "p50_us": float(np.percentile(us, 50)), "p99_us": float(np.percentile(us, 99)),
+            "reps": reps, "launches_per_call": 2, "bitexact_vs_oracle": bool(ok),
+            "oracle_us_per_call": t_or, "oracle_cores": orc.num_threads()}
 
 
 def cpu_baseline(budget_s=12.0):
@@ -557,6 +627,7 @@ def main():
         result["metric"] = f"secure {TASK} training samples/s (secondary config; headline metric is the MLP)"
     if rank == 0 and world == 1 and not args.no_ring_gemm:
         result["ring_gemm"] = [ring_gemm_figure(4096, 64), ring_gemm_figure(4096, 32)]
+        result["beaver_matmul_cfg1"] = beaver_latency_figure()
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         result["cpu_baseline"] = cpu_baseline()
     if rank == 0:

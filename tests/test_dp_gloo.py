@@ -101,3 +101,16 @@ def test_dp_update_shift_and_rows():
         start = pair_rows(step, pair, 4, 128, 60000)
         X, _ = synth.batch("mlp", step, 128, pair=pair, n_pairs=4)
         assert np.array_equal(X, synth.rows("mnist", start, 128))
+
+
+def test_split_pair_layout():
+    """Split deployment placement (SURVEY 8(e)): pair k = (rank k: party 0, rank k + N/2: party 1);
+    each rank's peer is the other party of its pair; odd world sizes are rejected."""
+    from paper_conf_icpp_chenzzzz020_b200.parallel import pair_layout
+    of = pair_layout(8)
+    assert [of(r) for r in range(8)] == [(0, 0, 4), (0, 1, 5), (0, 2, 6), (0, 3, 7),
+                                         (1, 0, 0), (1, 1, 1), (1, 2, 2), (1, 3, 3)]
+    assert pair_layout(2)(1) == (1, 0, 0)
+    for bad in (1, 3):
+        with pytest.raises(ValueError):
+            pair_layout(bad)
