@@ -333,8 +333,8 @@ psml_status psml_xport_exchange(psml_xport x, int32_t n, const void *const *send
 /* Bytes and exchanges issued through this transport so far (accounting for bench.py). */
 psml_status psml_xport_stats(psml_xport x, int64_t *bytes_sent, int64_t *exchanges);
 
-/* Party `party`'s half of one training step (LINREG / LOGREG / MLP; PSML_ERR_UNSUPPORTED for
- * CNN): X_i: batch x d_0, Y_i: batch x d_L, this party's shares (device).  The model's dealer
+/* Party `party`'s half of one training step (LINREG / LOGREG / MLP / CNN): X_i: batch x d_0
+ * (CNN: batch x C*H*W), Y_i: batch x d_L, this party's shares (device).  The model's dealer
  * pool must hold the step's material (psml_model_deal; in this simulation each party's process
  * runs the dealer and reads only its own half -- a deployment ships it from the client).
  * Leaves this party's untruncated weight-gradient share in psml_model_grads()[party] and its

@@ -228,6 +228,39 @@ struct ConvBeaverOps {
     }
 };
 
+// Split deployment, one party: E = mE0 + mE1 (this party's message + the peer's), F likewise;
+// C = im2col([party.E + U_X | E]) (.^T) . [F ; V] + Z, truncated (same arithmetic as above).
+template <typename T>
+struct ConvBeaverOps1 {
+    const T *mE0, *mE1, *UX, *mF0, *mF1, *V, *Z;
+    T *C;
+    ConvGeom g;
+    int64_t M, N, K, Kext;
+    int transposed, trunc, party;
+    static constexpr int nparty = 1;
+    __device__ __forceinline__ int64_t src(int64_t r, int64_t c) const { return conv_src(g, r, c); }
+    __device__ __forceinline__ T a(int, int64_t m, int64_t k) const {
+        const bool first = k < K;
+        const int64_t kk = first ? k : k - K;
+        const int64_t s = transposed ? src(kk, m) : src(m, kk);
+        const T e = mE0[s] + mE1[s], u = UX[s];
+        return first ? (T)((T)party * e + u) : e;
+    }
+    __device__ __forceinline__ T b(int, int64_t k, int64_t n) const {
+        const bool first = k < K;
+        const int64_t kk = first ? k : k - K, i = kk * N + n;
+        const T x = *(first ? mF0 + i : V + i), y = mF1[i];
+        return first ? (T)(x + y) : x;
+    }
+    __device__ __forceinline__ T zload(int, int64_t m, int64_t n) const { return Z[m * N + n]; }
+    __device__ __forceinline__ void put(int, int64_t m, int64_t n, T acc, T z) const {
+        C[m * N + n] = trunc_share<T>(acc + z, party, trunc);
+    }
+    __device__ __forceinline__ void store(int, int64_t m, int64_t n, T acc) const {
+        C[m * N + n] = trunc_share<T>(acc + Z[m * N + n], party, trunc);
+    }
+};
+
 // Dealer for the conv triplet: Z = im2col(U_0+U_1) (.^T) . (V_0+V_1), Z_1 = Z - PRG("Z0").
 template <typename T>
 struct ConvDealerOps {
@@ -546,7 +579,9 @@ psml_status launch_ring_gemm(const Ops &ops, T *ws, int64_t ws_words, cudaStream
     // the 16 x 16 small-tile kernel for small outputs or skinny outputs with many rows (CNN conv
     // im2col GEMMs), the 64 x 64 register-blocked kernel otherwise.
     const bool gemv = N <= 2 && M * Ops::nparty <= 4096 && Kx <= 8192;
-    if (!gemv && M * N * Ops::nparty <= ((int64_t)1 << 19) && simt_cl_enabled()) {
+    // the cluster kernel splits K at most 8 ways: very deep products with few output tiles (the
+    // CNN conv weight gradient, 75 x 200704 x 16) go to the small-tile kernel's deep split-K
+    if (!gemv && M * N * Ops::nparty <= ((int64_t)1 << 19) && Kx <= 32768 && simt_cl_enabled()) {
         ProfScope prof(PROF_GEMM, stream, (double)M * N * Kx * Ops::nparty);
         return launch_ring_gemm_cl<T, Ops>(ops, stream, sm_count);
     }

@@ -929,8 +929,53 @@ static psml_status party_had(PartyRun &r, const T *a, const T *b, int layer, int
     return PSML_OK;
 }
 
+// Conv Beaver product (R17): mask the un-expanded input, exchange, open inside the im2col GEMM.
+static psml_status party_conv(PartyRun &r, const T *X, const T *Bm, int transposed, int trunc, T *C) {
+    psml_model_s *m = r.m;
+    DealItem *it = find_item(m, 0, transposed ? OP_GRADW : OP_FWD, 0);
+    if (!it) return fail(PSML_ERR_STATE, "missing conv triplet");
+    const int64_t nin = m->B * m->g.C * m->g.H * m->g.W, K = it->K, N = it->N;
+    T *Es = m->ws, *Fs = Es + nin, *Er = Fs + K * N, *Fr = Er + nin, *partial = Fr + K * N;
+    const int64_t pw = m->ws_words - (partial - m->ws);
+    if (pw < it->M * N) return fail(PSML_ERR_STATE, "party workspace too small (conv)");
+    PSML_TRY(conv_mask_party<T>(X, Bm, it->U.p[r.p], it->V.p[r.p], m->B, m->g, K, N, Es, Fs, r.s));
+    PSML_TRY(xchg(r, {{Es, Er, nin}, {Fs, Fr, K * N}}));
+    return conv_open_party<T>(r.p, Es, Er, Fs, Fr, it->U.p[r.p], it->V.p[r.p], it->Z.p[r.p], m->B, m->g, transposed,
+                              N, trunc, C, partial, pw, r.s, m->ctx->sm_count);
+}
+
+static psml_status party_relu(PartyRun &r, const T *x, int layer, T *y, T *dr) {
+    DealItem *mat = find_item(r.m, layer, OP_RELU_MSB, 0), *h = find_item(r.m, layer, OP_HADAMARD, 0);
+    if (!mat || !h) return fail(PSML_ERR_STATE, "missing ReLU material");
+    return party_chain(r, x, mat, h, 1, y, dr, nullptr, nullptr);
+}
+
+static psml_status party_cnn(PartyRun &r, const T *X, const T *Y) {
+    psml_model_s *m = r.m;
+    const int F = m->ctx->ring.frac_bits;
+    const int p = r.p;
+    m->act[0].p[p] = (T *)X;
+    PSML_TRY(party_conv(r, X, m->W[0].p[p], 0, F, m->z[0].p[p]));
+    PSML_TRY(party_relu(r, m->z[0].p[p], 0, m->act[1].p[p], m->drelu[0].p[p]));
+    PSML_TRY(party_mm(r, m->act[1].p[p], m->W[1].p[p], 1, OP_FWD, 0, F, m->z[1].p[p]));
+    PSML_TRY(party_relu(r, m->z[1].p[p], 1, m->act[2].p[p], m->drelu[1].p[p]));
+    PSML_TRY(party_mm(r, m->act[2].p[p], m->W[2].p[p], 2, OP_FWD, 0, F, m->z[2].p[p]));
+    DealItem *mat = find_item(m, 2, OP_EQ9_MSB, 0), *h = find_item(m, 2, OP_HADAMARD, 2);
+    if (!mat || !h) return fail(PSML_ERR_STATE, "missing Eq. 9 material");
+    PSML_TRY(party_chain(r, m->z[2].p[p], mat, h, 2, m->yhat.p[p], nullptr, Y, m->delta.p[p]));
+    T *g[2];
+    PSML_TRY(party_mm(r, m->act[2].p[p], m->delta.p[p], 2, OP_GRADW, PSML_TRANS_A, 0, gradp(m, 2, g)[p]));
+    PSML_TRY(party_mm(r, m->delta.p[p], m->W[2].p[p], 2, OP_GRADIN, PSML_TRANS_B, F, m->tmp.p[p]));
+    PSML_TRY(party_had(r, m->tmp.p[p], m->drelu[1].p[p], 1, 1, m->delta.p[p]));
+    PSML_TRY(party_mm(r, m->act[1].p[p], m->delta.p[p], 1, OP_GRADW, PSML_TRANS_A, 0, gradp(m, 1, g)[p]));
+    PSML_TRY(party_mm(r, m->delta.p[p], m->W[1].p[p], 1, OP_GRADIN, PSML_TRANS_B, F, m->tmp.p[p]));
+    PSML_TRY(party_had(r, m->tmp.p[p], m->drelu[0].p[p], 0, 1, m->delta.p[p]));
+    return party_conv(r, m->act[0].p[p], m->delta.p[p], 1, 0, gradp(m, 0, g)[p]);
+}
+
 static psml_status party_forward_backward(PartyRun &r, const T *X, const T *Y) {
     psml_model_s *m = r.m;
+    if (m->d.kind == PSML_CNN) return party_cnn(r, X, Y);
     const int F = m->ctx->ring.frac_bits;
     const int p = r.p, nl = m->nl;
     const int64_t B = m->B;
@@ -1356,7 +1401,6 @@ psml_status psml_party_forward_backward(psml_model m, int32_t party, psml_xport 
                                         uint32_t step_id, psml_stream stream) {
     if (!m || !x) return fail(PSML_ERR_INVALID, "null model or transport");
     if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
-    if (m->d.kind == PSML_CNN) return fail(PSML_ERR_UNSUPPORTED, "split deployment: CNN not built (DESIGN.md §9)");
     PSML_TRY(check_ptrs({X_i, Y_i}));
     const int pool = (int)(step_id & 1);
     if (m->dealt_step[pool] != (int64_t)step_id || !m->dealt_full[pool])

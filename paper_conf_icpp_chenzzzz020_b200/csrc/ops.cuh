@@ -163,6 +163,33 @@ psml_status conv_beaver(const T *const X[2], const T *const Bm[2], const T *cons
     return launch_ring_gemm<T, ConvBeaverOps<T>>(ops, partial, ws_words - (partial - ws), s, sm_count);
 }
 
+// Split deployment, one party: round 1 writes this party's messages (E_send over the un-expanded
+// input, F_send); the caller exchanges them; round 2 opens them inside the im2col GEMM.
+template <typename T>
+psml_status conv_mask_party(const T *X, const T *Bm, const T *UX, const T *V, int64_t batch, ConvGeom g, int64_t K,
+                            int64_t N, T *Es, T *Fs, cudaStream_t s) {
+    MaskJobs<T> jobs;
+    jobs.j[0] = {X, UX, Es, batch, (int64_t)g.C * g.H * g.W, 0};
+    jobs.j[1] = {Bm, V, Fs, K, N, 0};
+    jobs.count = 2;
+    const int64_t maxt = std::max(((batch + 31) / 32) * (((int64_t)g.C * g.H * g.W + 31) / 32), ((K + 31) / 32) * ((N + 31) / 32));
+    mask_kernel<T><<<dim3((unsigned)std::min<int64_t>(maxt, 148 * 8), 1, 2), dim3(32, 8), 0, s>>>(jobs);
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
+template <typename T>
+psml_status conv_open_party(int party, const T *Es, const T *Er, const T *Fs, const T *Fr, const T *UX, const T *V,
+                            const T *Z, int64_t batch, ConvGeom g, int transposed, int64_t N, int trunc, T *C,
+                            T *partial, int64_t partial_words, cudaStream_t s, int sm_count) {
+    const int64_t rows = batch * g.OH * g.OW, kk = (int64_t)g.C * g.k * g.k;
+    ConvBeaverOps1<T> ops;
+    ops.mE0 = Es; ops.mE1 = Er; ops.mF0 = Fs; ops.mF1 = Fr; ops.UX = UX; ops.V = V; ops.Z = Z; ops.C = C;
+    ops.g = g; ops.M = transposed ? kk : rows; ops.N = N; ops.K = transposed ? rows : kk; ops.Kext = 2 * ops.K;
+    ops.transposed = transposed; ops.trunc = trunc; ops.party = party;
+    return launch_ring_gemm<T, ConvBeaverOps1<T>>(ops, partial, partial_words, s, sm_count);
+}
+
 template <typename T>
 inline int64_t conv_ws_words(int64_t batch, ConvGeom g, int transposed, int64_t N) {
     const int64_t nin = batch * g.C * g.H * g.W;

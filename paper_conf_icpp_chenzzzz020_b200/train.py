@@ -154,8 +154,6 @@ class PartyTrainer(SecureTrainer):
     material (the offline phase a deployment ships from the client)."""
 
     def __init__(self, task, W_init, party, transport, batch=128, pair_id=0, **kw):
-        if task == "cnn":
-            raise NotImplementedError("split deployment of the CNN is not built (DESIGN.md §9)")
         super().__init__(task, W_init, batch=batch, pair_id=pair_id, **kw)
         self.party = party
         self.xport = transport

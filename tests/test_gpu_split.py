@@ -119,7 +119,7 @@ def test_split_compressed_transmission(tmp_path):
 # library's transport -- here the host-staged gloo callback.  Each party's master-weight share
 # must equal the oracle's simulation of both parties (oracle/protocol.py) after every step.
 # ---------------------------------------------------------------------------------------------
-SPLIT_TASKS = [("linreg", 2), ("logreg", 2), ("mlp", 2)]
+SPLIT_TASKS = [("linreg", 2), ("logreg", 2), ("mlp", 2), ("cnn", 1)]
 
 
 def _party_train(rank, port, outdir):
