@@ -49,6 +49,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--task", default="mlp", choices=sorted(WORKLOADS),
                     help="headline is mlp (BASELINE metric); others are secondary configs")
+    ap.add_argument("--sweep", default=None, metavar="N1,N2,...",
+                    help="config-5 ring GEMM sweep (e.g. 512,1024,2048,4096,8192); prints JSON lines")
     ap.add_argument("--deployment", default="coresident", choices=["coresident", "split"],
                     help="coresident: both parties of a pair on one GPU (default); split: party 0 "
                          "and party 1 on different GPUs (ranks k and k + N/2), every opening "
@@ -572,6 +574,77 @@ def beaver_latency_figure(reps=2000):
             "oracle_us_per_call": t_or, "oracle_cores": orc.num_threads()}
 
 
+def tev(fn, reps):
+    import torch
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+    fn()
+    ts = []
+    for _ in range(reps):
+        flush.zero_()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        fn()
+        b.record()
+        torch.cuda.synchronize()
+        ts.append(a.elapsed_time(b))
+    return sorted(ts)[len(ts) // 2]
+
+
+def cfg5_sweep(ns):
+    """BASELINE config 5 sweep (bench.py --sweep): plain ring GEMM n^3 for l = 64 / 32 on tcgen05 (CUDA
+    cores to 2048), the co-resident Beaver secure matmul at every n, and -- the cpu_baseline leg --
+    the CPU oracle's ring matmul (all host threads) at n <= 2048 with bit-exact parity of the GPU
+    result, n^3-extrapolated above (labelled).  One JSON line per (n, l)."""
+    import numpy as np
+    import torch
+    from oracle import core as orc
+    from paper_conf_icpp_chenzzzz020_b200 import psml
+    oracle_t = {}
+    for n in ns:
+        for l in (64, 32):
+            pairs = 36 if l == 64 else 10
+            ring = psml.Ring(l, 13)
+            A = psml.prg_fill(ring, 1, psml.tag("bA"), 0, n * n).view(n, n)
+            B = psml.prg_fill(ring, 1, psml.tag("bB"), 0, n * n).view(n, n)
+            C = psml.empty(0, l, (n, n))
+            reps = 5 if n >= 4096 else 10
+            row = {"n": n, "l": l}
+            for be, name in ((2, "tcgen05"), (1, "cuda_core")):
+                if be == 1 and n > 2048:
+                    continue
+                ctx = psml.Ctx(l=l, backend=be)
+                ms = tev(lambda: psml.ring_gemm(ctx, A, B, out=C), reps)
+                row[name + "_ms"] = ms
+                row[name + "_useful_tops"] = pairs * 2.0 * n ** 3 / ms / 1e9
+                if be == 2:
+                    row["frac_of_int8_spec"] = row[name + "_useful_tops"] / INT8_DENSE_PEAK_TOPS
+                ctx.close()
+            # co-resident Beaver secure matmul (both parties: mask, open, Eq. 8 GEMM, trunc)
+            ctx = psml.Ctx(l=l)
+            As = psml.share(ring, 7, 1, A)
+            Bs = psml.share(ring, 7, 2, B)
+            U, V, Z = psml.triplet_gen(ctx, 3, 0, n, n, n)
+            Cs = psml.empty_pair((n, n), l)
+            ms = tev(lambda: psml.secure_matmul(ctx, As, Bs, U, V, Z, n, n, n, trunc=13, out=Cs), reps)
+            row["beaver_ms"] = ms
+            row["beaver_useful_tops"] = 2 * 2 * pairs * 2.0 * n ** 3 / ms / 1e9   # 2 parties x K' = 2K
+            ctx.close()
+            if n <= 2048:
+                An, Bn = A.cpu().numpy(), B.cpu().numpy()
+                t0 = time.perf_counter()
+                W = orc.ring_matmul(An, Bn, l)
+                oracle_t[(n, l)] = time.perf_counter() - t0
+                psml.ring_gemm(psml.Ctx(l=l, backend=2), A, B, out=C)
+                row["bitexact_vs_oracle"] = bool(np.array_equal(C.cpu().numpy().astype(np.uint64), W))
+                row["oracle_s"] = oracle_t[(n, l)]
+            else:
+                base = max(k for k in oracle_t if k[1] == l)
+                row["oracle_s_extrapolated_n3"] = oracle_t[base] * (n / base[0]) ** 3
+            row["oracle_threads"] = orc.num_threads()
+            print(json.dumps(row), flush=True)
+
+
+
 def cpu_baseline(budget_s=12.0):
     """The oracle as it stands on this host: whole secure MLP training steps (batch 128)."""
     import oracle
@@ -625,6 +698,11 @@ def main():
         out = bench_reference(args)
         if out is not None:
             print(json.dumps(out), flush=True)
+        return
+    if args.sweep:
+        from paper_conf_icpp_chenzzzz020_b200 import build
+        build.build()
+        cfg5_sweep([int(x) for x in args.sweep.split(",")])
         return
     if args.deployment == "split":
         result, rank = bench_split(args)

@@ -1,6 +1,6 @@
-"""Per-layer drift of the secure CNN vs fp64 SGD over one epoch (diagnostic)."""
+"""Per-layer drift of the secure CNN vs fp64 SGD over one epoch (diagnostic; test-side analysis, so it may use oracle/)."""
 import os, sys
-sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__)))))
 import numpy as np, torch
 import synth
 from oracle import plain
