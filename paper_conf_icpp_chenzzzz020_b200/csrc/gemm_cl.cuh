@@ -30,25 +30,7 @@ struct ClCfg {
 };
 using ClDefault = ClCfg<32, 32, 256, 2, 2, 16>;   // measured best on the MLP shapes (tools/micro)
 
-// ring multiply-accumulate with split accumulators for u64
-template <typename T> struct RingAcc {
-    T v;
-    __device__ __forceinline__ void zero() { v = 0; }
-    __device__ __forceinline__ void mac(T a, T b) { v += a * b; }
-    __device__ __forceinline__ T value() const { return v; }
-};
-template <> struct RingAcc<uint64_t> {
-    uint64_t w;        // sum of lo.lo (64-bit, IMAD.WIDE.U32 with accumulate)
-    uint32_t x1, x2;   // sums of lo.hi and hi.lo (mod 2^32), two chains
-    __device__ __forceinline__ void zero() { w = 0; x1 = 0; x2 = 0; }
-    __device__ __forceinline__ void mac(uint64_t a, uint64_t b) {
-        const uint32_t al = (uint32_t)a, ah = (uint32_t)(a >> 32), bl = (uint32_t)b, bh = (uint32_t)(b >> 32);
-        asm("mad.wide.u32 %0, %1, %2, %0;" : "+l"(w) : "r"(al), "r"(bl));
-        asm("mad.lo.u32 %0, %1, %2, %0;" : "+r"(x1) : "r"(al), "r"(bh));
-        asm("mad.lo.u32 %0, %1, %2, %0;" : "+r"(x2) : "r"(ah), "r"(bl));
-    }
-    __device__ __forceinline__ uint64_t value() const { return w + ((uint64_t)(x1 + x2) << 32); }
-};
+// RingAcc (split-accumulator ring MAC) lives in gemm_simt.cuh, which includes this file.
 
 template <typename T, class Ops, class C>
 __device__ __forceinline__ void cl_tile(const Ops &ops, int p, int64_t m0, int64_t n0, int64_t kbeg, int64_t kend,

@@ -18,6 +18,26 @@
 
 namespace psml {
 
+// ring multiply-accumulate with split accumulators for u64
+template <typename T> struct RingAcc {
+    T v;
+    __device__ __forceinline__ void zero() { v = 0; }
+    __device__ __forceinline__ void mac(T a, T b) { v += a * b; }
+    __device__ __forceinline__ T value() const { return v; }
+};
+template <> struct RingAcc<uint64_t> {
+    uint64_t w;        // sum of lo.lo (64-bit, IMAD.WIDE.U32 with accumulate)
+    uint32_t x1, x2;   // sums of lo.hi and hi.lo (mod 2^32), two chains
+    __device__ __forceinline__ void zero() { w = 0; x1 = 0; x2 = 0; }
+    __device__ __forceinline__ void mac(uint64_t a, uint64_t b) {
+        const uint32_t al = (uint32_t)a, ah = (uint32_t)(a >> 32), bl = (uint32_t)b, bh = (uint32_t)(b >> 32);
+        asm("mad.wide.u32 %0, %1, %2, %0;" : "+l"(w) : "r"(al), "r"(bl));
+        asm("mad.lo.u32 %0, %1, %2, %0;" : "+r"(x1) : "r"(al), "r"(bh));
+        asm("mad.lo.u32 %0, %1, %2, %0;" : "+r"(x2) : "r"(ah), "r"(bl));
+    }
+    __device__ __forceinline__ uint64_t value() const { return w + ((uint64_t)(x1 + x2) << 32); }
+};
+
 // ---------------------------------------------------------------------------------------------
 // operand/epilogue policies.  Each provides:
 //   nparty, M, N, Kext; T a(p, m, k); T b(p, k, n); void store(p, m, n, T acc)
@@ -536,6 +556,40 @@ __global__ void __launch_bounds__(256) ring_gemv(Ops ops, int64_t k_per_split, i
     }
 }
 
+// Tall-skinny products (N <= NN = 16, short K'; the CNN conv im2col GEMMs, 100352 x 150 x 16):
+// one thread per output row holding all N accumulators, the whole K' x N B operand staged in
+// shared memory once per CTA (read as a broadcast), A gathered per (row, k) straight from the
+// producers' buffers (consecutive rows = consecutive output pixels: coalesced).
+template <typename T, class Ops, int NN>
+__global__ void __launch_bounds__(256) ring_gemm_rows(Ops ops) {
+    extern __shared__ __align__(16) unsigned char rows_smem[];
+    T *Bs = reinterpret_cast<T *>(rows_smem);   // [Kext][NN]
+    const int p = blockIdx.y;
+    const int64_t Kx = ops.Kext;
+    const int N = (int)ops.N;
+    for (int64_t i = threadIdx.x; i < Kx * NN; i += blockDim.x) {
+        const int64_t k = i / NN;
+        const int n = (int)(i % NN);
+        Bs[i] = n < N ? ops.b(p, k, n) : (T)0;
+    }
+    __syncthreads();
+    const int64_t m = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (m >= ops.M) return;
+    RingAcc<T> acc[NN];
+#pragma unroll
+    for (int j = 0; j < NN; ++j) acc[j].zero();
+#pragma unroll 2
+    for (int64_t k = 0; k < Kx; ++k) {
+        const T a = ops.a(p, m, k);
+        const T *b = Bs + k * NN;
+#pragma unroll
+        for (int j = 0; j < NN; ++j) acc[j].mac(a, b[j]);
+    }
+#pragma unroll
+    for (int j = 0; j < NN; ++j)
+        if (j < N) ops.store(p, m, j, acc[j].value());
+}
+
 template <typename T, class Ops>
 __global__ void ring_gemm_finalize(Ops ops, const T *__restrict__ partial) {
     const int64_t total = ops.M * ops.N * Ops::nparty;
@@ -562,6 +616,16 @@ inline bool simt_cl_enabled() {
     return v == 1;
 }
 
+// PSML_ROWS=0 keeps tall-skinny products on the 16 x 16 small-tile kernel.
+inline bool rows_kernel_enabled() {
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("PSML_ROWS");
+        v = (e && e[0] == '0') ? 0 : 1;
+    }
+    return v == 1;
+}
+
 // ---------------------------------------------------------------------------------------------
 // host-side dispatcher: picks kernel, tile and split-K; `ws` must hold nparty*M*N words when
 // split-K is chosen (ws_words reports the need; pass ws = nullptr to query).
@@ -584,6 +648,20 @@ psml_status launch_ring_gemm(const Ops &ops, T *ws, int64_t ws_words, cudaStream
     if (!gemv && M * N * Ops::nparty <= ((int64_t)1 << 19) && Kx <= 32768 && simt_cl_enabled()) {
         ProfScope prof(PROF_GEMM, stream, (double)M * N * Kx * Ops::nparty);
         return launch_ring_gemm_cl<T, Ops>(ops, stream, sm_count);
+    }
+    if (!gemv && N <= 16 && M * Ops::nparty >= 8192 && Kx * 16 * (int64_t)sizeof(T) <= 96 * 1024 &&
+        rows_kernel_enabled()) {
+        const size_t smem = (size_t)Kx * 16 * sizeof(T);
+        static bool attr = false;   // per (T, Ops) instantiation
+        if (!attr) {
+            PSML_CUDA_TRY(cudaFuncSetAttribute(ring_gemm_rows<T, Ops, 16>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                               96 * 1024));
+            attr = true;
+        }
+        ProfScope prof(PROF_GEMM, stream, (double)M * N * Kx * Ops::nparty);
+        ring_gemm_rows<T, Ops, 16><<<dim3((unsigned)((M + 255) / 256), Ops::nparty), 256, smem, stream>>>(ops);
+        PSML_LAUNCH_CHECK();
+        return PSML_OK;
     }
     const bool small = !gemv && (N <= 16 || M * N * Ops::nparty <= ((int64_t)1 << 18));
     int splits = 1;

@@ -357,6 +357,11 @@ static psml_status deal_item(psml_model_s *m, DealItem &it, uint32_t step, cudaS
 // Work lists of the fused dealer for items[pool] (step field of the call ids filled in on device).
 static psml_status build_plan(psml_model_s *m, int pool, bool infer_only) {
     DealPlan &P = m->plan[pool][infer_only ? 1 : 0];
+    {   // cluster split of the dealer's grouped Z = U V launch (PSML_DEAL_KS; default 4)
+        const char *e = getenv("PSML_DEAL_KS");
+        const int v = e ? atoi(e) : 4;
+        P.gemm_ks = (v == 1 || v == 2 || v == 4 || v == 8) ? v : 4;
+    }
     std::vector<PrgJob> pj;
     std::vector<ClJob<DealerOps<T>>> gj;
     auto job = [&](int kind, std::initializer_list<uint32_t> tags, uint64_t cid, int64_t n,

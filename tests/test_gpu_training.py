@@ -145,16 +145,18 @@ def test_explicit_mask_round_matches_fused_open():
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
 
 
-@pytest.mark.parametrize("mode", ["simt", "tc"])
-def test_seg_gemm_backends_match_oracle(mode):
+@pytest.mark.parametrize("env", [{"PSML_SEG": "simt"}, {"PSML_SEG": "tc"}, {"PSML_ROWS": "0"}],
+                         ids=["seg_simt", "seg_tc", "rows_off"])
+def test_seg_gemm_backends_match_oracle(env):
     """PSML_SEG=simt: every opened Beaver product of the training step on the CUDA-core
     two-segment GEMM; PSML_SEG=tc: every eligible one on the tcgen05 in-kernel-split GEMM
-    (gemm_tcseg.cu; by default only groups of >= 2^25 ring MACs go there).  Both reproduce the
-    oracle exactly."""
+    (gemm_tcseg.cu; by default only groups of >= 2^25 ring MACs go there); PSML_ROWS=0: the CNN's
+    tall-skinny conv products on the 16 x 16 small-tile kernel instead of ring_gemm_rows.  All
+    reproduce the oracle exactly."""
     import os
     import subprocess
     import sys
-    env = dict(os.environ, PSML_SEG=mode)
+    env = dict(os.environ, **env)
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
     r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu", "-k",
                         "training_bitexact_vs_oracle or graph_replay or secure_matmul_bitexact",
