@@ -319,6 +319,9 @@ def bench_ours(args):
         psml.prof_enable(cls)
         psml.prof_read()
         for i in range(K):
+            # a GPU sleep ahead of each step lets the host enqueue the whole step first, so the
+            # per-launch events bracket device time, not host submission gaps
+            torch.cuda._sleep(3_000_000)
             one_step(base + i, Xs[i % nb], Ys[i % nb])
         ms, n, work = psml.prof_read()
         psml.prof_enable(-1)

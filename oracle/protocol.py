@@ -57,6 +57,40 @@ def trunc_pair(x, d):
     return core.truncate(x[0], 0, d), core.truncate(x[1], 1, d)
 
 
+# ---------------------------------------------------------------------------------------------
+# Diagnostics: the oracle knows the plaintext, so it counts SecureML
+# truncation failures (|t - floor(x / 2^d)| > 1, R7: probability <= 2^(l_x + 1 - l) each) and
+# secure-comparison mismatches (DReLU != [x >= 0], Eq. 9 output != clamp(x + 1/2, 0, 1), R8/R9).
+# A fixed-seed run must report 0 of each.  Off by default (costs a reconstruction per check).
+# ---------------------------------------------------------------------------------------------
+DIAG = {"on": False, "trunc_checked": 0, "trunc_fail": 0, "msb_checked": 0, "msb_fail": 0}
+
+
+def diag_reset(on=True):
+    DIAG.update(on=on, trunc_checked=0, trunc_fail=0, msb_checked=0, msb_fail=0)
+
+
+def _signed(v):
+    return np.asarray(v, dtype=np.uint64).view(np.int64)
+
+
+def check_trunc(pre, post, d):
+    """Count elements whose truncated reconstruction is more than 1 LSB from floor(x / 2^d)."""
+    if not DIAG["on"] or d == 0:
+        return
+    x = _signed(pre[0] + pre[1])
+    t = _signed(post[0] + post[1])
+    diff = t - (x >> np.int64(d))          # int64 wraparound keeps a failure far outside [-1, 1]
+    DIAG["trunc_checked"] += int(x.size)
+    DIAG["trunc_fail"] += int(np.count_nonzero((diff > 1) | (diff < -1)))
+
+
+def checked_trunc(x, d):
+    t = trunc_pair(x, d)
+    check_trunc(x, t, d)
+    return t
+
+
 def sub_pair(a, b):
     return a[0] - b[0], a[1] - b[1]
 
@@ -88,7 +122,8 @@ def matmul(A, B, pair, step, layer, op, trunc):
     M, K = A[0].shape
     N = B[0].shape[1]
     trip = core.triplet_gen(DEALER_SEED, call_id(pair, step, layer, op, 0), M, K, N, L)
-    return core.beaver_matmul(A, B, trip, trunc=trunc, l=L)
+    c = core.beaver_matmul(A, B, trip, trunc=0, l=L)   # Eq. 6/8, then truncation (R7)
+    return checked_trunc(c, trunc) if trunc else c
 
 
 def relu(z, pair, step, layer):
@@ -96,6 +131,11 @@ def relu(z, pair, step, layer):
     mat = core.msb_dealer(DEALER_SEED, call_id(pair, step, layer, OP_RELU_MSB, 0), n, L)
     ht = core.hadamard_triplet_gen(DEALER_SEED, call_id(pair, step, layer, OP_HADAMARD, 0), n, L)
     (r0, r1), (d0, d1) = core.secure_relu((z[0].reshape(-1), z[1].reshape(-1)), mat, ht, L)
+    if DIAG["on"]:   # DReLU = 1 - MSB(x) must equal [x >= 0] on the plaintext
+        x = _signed(z[0].reshape(-1) + z[1].reshape(-1))
+        dr = np.asarray(d0 + d1, dtype=np.uint64)
+        DIAG["msb_checked"] += int(x.size)
+        DIAG["msb_fail"] += int(np.count_nonzero(dr != (x >= 0).astype(np.uint64)))
     s = z[0].shape
     return (r0.reshape(s), r1.reshape(s)), (d0.reshape(s), d1.reshape(s))
 
@@ -104,7 +144,13 @@ def eq9(z, pair, step, layer):
     n = z[0].size
     mat = core.msb_dealer(DEALER_SEED, call_id(pair, step, layer, OP_EQ9_MSB, 0), 2 * n, L)
     ht = core.hadamard_triplet_gen(DEALER_SEED, call_id(pair, step, layer, OP_HADAMARD, 2), 2 * n, L)
-    return core.secure_eq9(z, mat, ht, L, F)
+    y = core.secure_eq9(z, mat, ht, L, F)
+    if DIAG["on"]:   # Eq. 9 on the grid: clamp(x + 2^(F-1), 0, 2^F) exactly (R8)
+        x = _signed(z[0] + z[1])
+        want = np.clip(x + (1 << (F - 1)), 0, 1 << F)
+        DIAG["msb_checked"] += int(x.size)
+        DIAG["msb_fail"] += int(np.count_nonzero(_signed(y[0] + y[1]) != want))
+    return y
 
 
 def hadamard(a, b, pair, step, layer, slot):
@@ -147,8 +193,8 @@ def conv_matmul(X, Bm, U, V, Z, transpose, trunc):
     out = []
     for i in range(2):
         c = i * EF + core.ring_matmul(Ec, V[i]) + core.ring_matmul(tr(col(U[i])), Fm) + Z[i]
-        out.append(core.truncate(c, i, trunc) if trunc else c)
-    return tuple(out)
+        out.append(c)
+    return checked_trunc(tuple(out), trunc) if trunc else tuple(out)
 
 
 # ---------------------------------------------------------------------------------------------
@@ -217,9 +263,9 @@ def apply_update(model, grads, n_pairs=1):
     extra = int(np.log2(n_pairs))
     assert (1 << extra) == n_pairs
     for layer, g in enumerate(grads):
-        gt = trunc_pair(g, 26 + LR_SHIFT - MASTER + extra)
+        gt = checked_trunc(g, 26 + LR_SHIFT - MASTER + extra)
         model.Wm[layer] = sub_pair(model.Wm[layer], gt)
-        model.W[layer] = trunc_pair(model.Wm[layer], MASTER - F)
+        model.W[layer] = checked_trunc(model.Wm[layer], MASTER - F)
 
 
 def train_step(model, X, Y, step, pair=0):

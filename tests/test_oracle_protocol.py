@@ -70,3 +70,32 @@ def test_oracle_inference_matches_plaintext_forward():
     got = core.decode(core.reconstruct(*yh))
     want = pm.forward(plain.q(X, P.F))[2]
     assert np.abs(got - want).max() < 2.0 ** -9
+
+
+def test_diagnostics_zero_failures_and_checker_pinned():
+    """a fixed-seed run reports 0 SecureML truncation failures and 0 secure
+    comparison mismatches (DReLU vs [x >= 0], Eq. 9 vs clamp(x + 1/2, 0, 1)).  The checker itself
+    is pinned: a skipped truncation is counted, a correct SecureML truncation is not."""
+    P.diag_reset(True)
+    try:
+        for task, steps in (("mlp", 2), ("logreg", 2)):
+            m = P.Model(task, synth.init_weights(task))
+            for s in range(steps):
+                X, Y = synth.batch(task, s)
+                P.train_step(m, X, Y, s)
+        d = dict(P.DIAG)
+        assert d["trunc_checked"] > 100_000 and d["msb_checked"] > 30_000, d
+        assert d["trunc_fail"] == 0 and d["msb_fail"] == 0, d
+        # checker pins: an untruncated "result" is far from floor(x / 2^13) ...
+        P.diag_reset(True)
+        x = (np.array([5 << 20, (1 << 64) - (7 << 20)], dtype=np.uint64), np.zeros(2, dtype=np.uint64))
+        P.check_trunc(x, x, 13)
+        assert P.DIAG["trunc_fail"] == 2
+        # ... while SecureML's own truncation of a shared value passes (x split with random share)
+        r = np.array([0x123456789ABCDEF0, 0x0FEDCBA987654321], dtype=np.uint64)
+        y = (r, x[0] - r)
+        P.diag_reset(True)
+        P.check_trunc(y, P.trunc_pair(y, 13), 13)
+        assert P.DIAG["trunc_fail"] == 0 and P.DIAG["trunc_checked"] == 2
+    finally:
+        P.diag_reset(False)
