@@ -331,6 +331,7 @@ def bench_ours(args):
                          "ms_per_launch": ms / max(n, 1)}
     result["kernel_classes"] = classes
     result["roofline"] = roofline(classes, result["clocks"])
+    result["offline"] = offline_figure(classes["dealer"], samples / K)
     return result, tr, world, rank
 
 
@@ -481,6 +482,23 @@ def _roofline(classes, clocks):
             "frac": ach / peak, "traffic": None,
             "peak_source": "measured" if "hbm_gbs" in mp else "fallback",
             "selection": "largest online-phase kernel class (dealer overlapped)"}
+
+
+def offline_figure(dealer, samples_per_step):
+    """Offline phase (Table 3): the dealer's material for one step --
+    ChaCha20 streams (U/V/Z_0 masks, AND triplets, daBits, Hadamard triplets) plus the grouped
+    Z_1 = U V - Z_0 products -- timed alone (class 'dealer').  The PRG is bound by the ALU pipe:
+    a ChaCha20 block is 80 quarter rounds x (4 LOP3 + 4 SHF) = 640 ALU-pipe ops (the 4 adds per
+    quarter round issue as IMAD on the FMA pipe, cuobjdump of deal_prg_kernel); ALU-pipe peak =
+    148 SMs x 64 lanes/clk x 1965 MHz (B300_MICROARCH: alu rt_SMSP = 2).  The class time includes
+    the Z = U V products, so the fraction is a lower bound for the PRG kernel."""
+    sec = dealer["ms_per_step"] / 1e3
+    blocks = dealer["work_per_launch"] * dealer["launches_per_step"]
+    peak_blocks = 148 * 64 * 1.965e9 / 640
+    return {"ms_per_step": dealer["ms_per_step"], "samples_per_s": samples_per_step / sec,
+            "chacha20_blocks_per_step": blocks, "prg_output_GBps": blocks * 64 / sec / 1e9,
+            "prg_alu_roofline": {"bound": "alu", "achieved": blocks / sec / 1e9, "peak": peak_blocks / 1e9,
+                                 "unit": "G ChaCha20 blocks/s", "frac_lower_bound": blocks / sec / peak_blocks}}
 
 
 def int8_peak_tops():

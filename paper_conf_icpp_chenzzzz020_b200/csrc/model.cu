@@ -91,6 +91,9 @@ struct DealPlan {   // fused dealer of one pool (full or inference-only)
     PrgJob *prg = nullptr;
     int n_prg = 0;
     int64_t prg_blocks = 0;
+    int n_prg_mat = 0;           // jobs [0, n_prg_mat) = matrix-triplet streams (U, V, Z_0), needed
+    int64_t prg_mat_blocks = 0;  // by the Z = U V launch; the rest (AND/daBit/Hadamard) after them
+    double chacha_blocks = 0;   // ChaCha20 block evaluations of the PRG work list (all streams)
     ClJob<DealerOps<T>> *gemm = nullptr;
     int n_gemm = 0, gemm_ks = 4;
     int64_t gemm_tiles = 0;
@@ -136,6 +139,11 @@ struct psml_model_s {
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
     cudaStream_t hi = nullptr;         // online phase inside the pipelined graph (highest priority)
     cudaEvent_t ev_hi = nullptr;
+    cudaEvent_t ev_late = nullptr;
+    cudaStream_t side2 = nullptr;      // second dealer branch (AND / daBit / Hadamard PRG streams)
+    cudaEvent_t ev_d2 = nullptr, ev_d2j = nullptr;     // late fork point of the dealer branch (PSML_DEAL_AFTER)
+    int deal_pending_pool = -1;        // capture in progress: dealer branch not forked yet
+    int deal_after = 0, deal_stage = 0;
 };
 
 namespace psml {
@@ -362,7 +370,7 @@ static psml_status build_plan(psml_model_s *m, int pool, bool infer_only) {
         const int v = e ? atoi(e) : 4;
         P.gemm_ks = (v == 1 || v == 2 || v == 4 || v == 8) ? v : 4;
     }
-    std::vector<PrgJob> pj;
+    std::vector<PrgJob> pjm, pjr;   // matrix-triplet streams, then the rest
     std::vector<ClJob<DealerOps<T>>> gj;
     auto job = [&](int kind, std::initializer_list<uint32_t> tags, uint64_t cid, int64_t n,
                    std::initializer_list<T *> outs) {
@@ -373,9 +381,9 @@ static psml_status build_plan(psml_model_s *m, int pool, bool infer_only) {
         for (uint32_t t : tags) j.tag[i++] = t;
         i = 0;
         for (T *o : outs) j.out[i++] = o;
-        j.cid = cid; j.n = n; j.blk_begin = P.prg_blocks;
-        P.prg_blocks += (n + 7) / 8;
-        pj.push_back(j);
+        j.cid = cid; j.n = n;
+        P.chacha_blocks += (double)((n + 7) / 8) * (double)tags.size();
+        (kind == PJ_PAIR || kind == PJ_SINGLE ? pjm : pjr).push_back(j);
     };
     const int L = 6;   // log2(64): 2L AND triplets + one daBit per element (R9)
     auto &items = m->items[pool];
@@ -422,6 +430,14 @@ static psml_status build_plan(psml_model_s *m, int pool, bool infer_only) {
         }
         }
     }
+    std::vector<PrgJob> pj(pjm);
+    pj.insert(pj.end(), pjr.begin(), pjr.end());
+    P.n_prg_mat = (int)pjm.size();
+    for (size_t i = 0; i < pj.size(); ++i) {
+        pj[i].blk_begin = P.prg_blocks;
+        P.prg_blocks += (pj[i].n + 7) / 8;
+        if ((int)i + 1 == P.n_prg_mat) P.prg_mat_blocks = P.prg_blocks;
+    }
     P.n_prg = (int)pj.size();
     P.n_gemm = (int)gj.size();
     if (P.n_prg) {
@@ -440,7 +456,39 @@ static psml_status build_plan(psml_model_s *m, int pool, bool infer_only) {
     return PSML_OK;
 }
 
-static psml_status deal_pool(psml_model_s *m, int pool, uint32_t step, bool infer_only, cudaStream_t s) {
+// second dealer branch inside a pipelined capture (PSML_DEAL_SPLIT=0: one branch)
+static cudaStream_t deal_s2(psml_model_s *m) {
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("PSML_DEAL_SPLIT");
+        v = (e && e[0] == '0') ? 0 : 1;
+    }
+    return v ? m->side2 : nullptr;
+}
+
+// PRG jobs [j0, j1) (blocks [b0, b1)) of plan P on stream s
+static psml_status deal_prg_launch(psml_model_s *m, const DealPlan &P, int j0, int j1, int64_t b0, int64_t b1,
+                                   cudaStream_t s) {
+    if (j1 <= j0 || b1 <= b0) return PSML_OK;
+    // a bounded grid (grid-stride): the PRG work runs beside the online phase instead of
+    // occupying every SM's register file ahead of it (PSML_DEAL_CTAS per SM; 0 = full grid)
+    static int per_sm = -1;
+    if (per_sm < 0) {
+        const char *e = getenv("PSML_DEAL_CTAS");
+        per_sm = e ? atoi(e) : 4;   // measured best of {1, 2, 4, full} (tools/gpu44.sh)
+    }
+    const int64_t full = (b1 - b0 + 127) / 128;
+    const int64_t grid = per_sm > 0 ? std::min<int64_t>(full, (int64_t)per_sm * m->ctx->sm_count) : full;
+    deal_prg_kernel<<<(unsigned)grid, 128, 0, s>>>(P.prg + j0, j1 - j0, b0, b1, m->d.dealer_seed, m->step_dev);
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
+// Dealer of one pool.  With a second stream s2 (the pipelined graph), the AND / daBit / Hadamard
+// streams run on s2 while s runs the matrix-triplet streams and then Z = U V, so the products'
+// material is ready early; s joins s2 before returning.
+static psml_status deal_pool(psml_model_s *m, int pool, uint32_t step, bool infer_only, cudaStream_t s,
+                             cudaStream_t s2 = nullptr) {
     if (!fused_deal()) {
         for (auto &it : m->items[pool]) {
             if (infer_only && !it.fwd) continue;
@@ -450,20 +498,17 @@ static psml_status deal_pool(psml_model_s *m, int pool, uint32_t step, bool infe
     }
     (void)step;   // the step field comes from m->step_dev (set by the caller / the graph)
     DealPlan &P = m->plan[pool][infer_only ? 1 : 0];
+    const bool fork = s2 && P.n_prg_mat > 0 && P.n_prg > P.n_prg_mat;
     {
-        ProfScope prof(PROF_DEALER, s, 0.0);
-        if (P.n_prg) {
-            // a bounded grid (grid-stride): the PRG work runs beside the online phase instead of
-            // occupying every SM's register file ahead of it (PSML_DEAL_CTAS per SM; 0 = full grid)
-            static int per_sm = -1;
-            if (per_sm < 0) {
-                const char *e = getenv("PSML_DEAL_CTAS");
-                per_sm = e ? atoi(e) : 4;   // measured best of {1, 2, 4, full} (tools/gpu44.sh)
-            }
-            const int64_t full = (P.prg_blocks + 127) / 128;
-            const int64_t grid = per_sm > 0 ? std::min<int64_t>(full, (int64_t)per_sm * m->ctx->sm_count) : full;
-            deal_prg_kernel<<<(unsigned)grid, 128, 0, s>>>(P.prg, P.n_prg, P.prg_blocks, m->d.dealer_seed, m->step_dev);
-            PSML_LAUNCH_CHECK();
+        ProfScope prof(PROF_DEALER, s, P.chacha_blocks);   // work = ChaCha20 blocks of the step
+        if (fork) {
+            PSML_CUDA_TRY(cudaEventRecord(m->ev_d2, s));
+            PSML_CUDA_TRY(cudaStreamWaitEvent(s2, m->ev_d2, 0));
+            PSML_TRY(deal_prg_launch(m, P, P.n_prg_mat, P.n_prg, P.prg_mat_blocks, P.prg_blocks, s2));
+            PSML_CUDA_TRY(cudaEventRecord(m->ev_d2j, s2));
+            PSML_TRY(deal_prg_launch(m, P, 0, P.n_prg_mat, 0, P.prg_mat_blocks, s));
+        } else {
+            PSML_TRY(deal_prg_launch(m, P, 0, P.n_prg, 0, P.prg_blocks, s));
         }
         if (P.n_gemm) {
             cudaLaunchConfig_t cfg = {};
@@ -480,6 +525,7 @@ static psml_status deal_pool(psml_model_s *m, int pool, uint32_t step, bool infe
         }
     }
     for (int k : P.rest) PSML_TRY(deal_gemm(m, m->items[pool][k], s));
+    if (fork) PSML_CUDA_TRY(cudaStreamWaitEvent(s, m->ev_d2j, 0));
     return PSML_OK;
 }
 
@@ -638,6 +684,22 @@ static psml_status alloc_open_bufs(psml_model_s *m) {
     return PSML_OK;
 }
 
+// Pipelined capture: the next step's dealer branch forks from the online chain after its
+// `deal_after`-th stage (0 = at the start of the step), so the dealer's persistent PRG CTAs do not
+// hold the SMs the first products need.
+static psml_status deal_fork_point(psml_model_s *m, cudaStream_t s, bool force = false) {
+    if (m->deal_pending_pool < 0) return PSML_OK;
+    if (!force && ++m->deal_stage < m->deal_after) return PSML_OK;
+    const int pool = m->deal_pending_pool;
+    m->deal_pending_pool = -1;
+    PSML_CUDA_TRY(cudaEventRecord(m->ev_late, s));
+    PSML_CUDA_TRY(cudaStreamWaitEvent(m->side, m->ev_late, 0));
+    PSML_TRY(deal_pool(m, pool, 0, false, m->side, deal_s2(m)));
+    PSML_CUDA_TRY(cudaEventRecord(m->ev_join, m->side));
+    return PSML_OK;
+}
+
+
 static psml_status fused_forward_backward(psml_model_s *m, const T *const X[2], const T *const Y[2], cudaStream_t s) {
     const int F = m->ctx->ring.frac_bits;
     const int nl = m->nl;
@@ -711,12 +773,14 @@ static psml_status fused_forward_backward(psml_model_s *m, const T *const X[2], 
         ProfScope prof(PROF_MASK, s, 0.0);
         PSML_CUDA_TRY(launch_pdl(open_list_kernel<T>, dim3((unsigned)tiles), dim3(32, 8), s, L));
         PSML_LAUNCH_CHECK();
+        PSML_TRY(deal_fork_point(m, s));
     }
     // 2. forward
     T *yo[2] = {m->yhat.p[0], m->yhat.p[1]};
     for (int l = 0; l < nl; ++l) {
         SegArgs<T> a = seg(l, OP_FWD, m->z[l].p[0], m->z[l].p[1], F);
         PSML_TRY(launch_seg_group<T>(&a, 1, s, m->ctx->sm_count));
+        PSML_TRY(deal_fork_point(m, s));
         const int64_t w = m->dims[l + 1];
         if (l < nl - 1) {
             Emits<T> em{};
@@ -728,6 +792,7 @@ static psml_status fused_forward_backward(psml_model_s *m, const T *const X[2], 
             PSML_TRY(msb_chain<T>(m->z[l].cp(), mat->n, mat->mat.cp(), 0, 0, 1, nullptr, nullptr, m->drelu[l].pp(),
                                   h->U.cp(), h->V.cp(), h->Z.cp(), m->act[l + 1].pp(), nullptr, nullptr, m->ws, s,
                                   &em));
+            PSML_TRY(deal_fork_point(m, s));
         } else {
             Emits<T> em{};
             em.e[0] = emitB(l, OP_GRADW, B, w);
@@ -759,6 +824,7 @@ static psml_status fused_forward_backward(psml_model_s *m, const T *const X[2], 
         jobs[0] = seg(l, OP_GRADW, g[0], g[1], 0);
         if (l > 0) jobs[1] = seg(l, OP_GRADIN, m->tmp.p[0], m->tmp.p[1], F);
         PSML_TRY(launch_seg_group<T>(jobs, l > 0 ? 2 : 1, s, m->ctx->sm_count));
+        PSML_TRY(deal_fork_point(m, s));
         if (l > 0) {
             DealItem *h = find_item(m, l - 1, OP_HADAMARD, 1);
             if (!h) return fail(PSML_ERR_STATE, "missing Hadamard triplet");
@@ -1122,11 +1188,15 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
         int lo = 0, hi = 0;
         PSML_CUDA_TRY(cudaDeviceGetStreamPriorityRange(&lo, &hi));
         PSML_CUDA_TRY(cudaStreamCreateWithPriority(&m->side, cudaStreamNonBlocking, lo));
+        PSML_CUDA_TRY(cudaStreamCreateWithPriority(&m->side2, cudaStreamNonBlocking, lo));
         PSML_CUDA_TRY(cudaStreamCreateWithPriority(&m->hi, cudaStreamNonBlocking, hi));
         PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_hi, cudaEventDisableTiming));
     }
     PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_fork, cudaEventDisableTiming));
     PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_join, cudaEventDisableTiming));
+    PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_late, cudaEventDisableTiming));
+    PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_d2, cudaEventDisableTiming));
+    PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_d2j, cudaEventDisableTiming));
     {
         T *sd = nullptr;
         PSML_TRY(dalloc(mp, &sd, 1));
@@ -1148,6 +1218,10 @@ psml_status psml_model_destroy(psml_model model) {
     if (model->hi) cudaStreamDestroy(model->hi);
     if (model->ev_hi) cudaEventDestroy(model->ev_hi);
     if (model->ev_join) cudaEventDestroy(model->ev_join);
+    if (model->ev_late) cudaEventDestroy(model->ev_late);
+    if (model->ev_d2) cudaEventDestroy(model->ev_d2);
+    if (model->ev_d2j) cudaEventDestroy(model->ev_d2j);
+    if (model->side2) cudaStreamDestroy(model->side2);
     for (void *p : model->allocs) cudaFree(p);
     delete model;
     return PSML_OK;
@@ -1294,14 +1368,27 @@ static psml_status capture_one(psml_model_s *m, int pool, const T *const X[2], c
             if (cudaStreamWaitEvent(m->hi, m->ev_fork, 0) != cudaSuccess) st = fail(PSML_ERR_CUDA, "graph fork failed");
             on = m->hi;
         }
-        if (st == PSML_OK) st = deal_pool(m, 1 - pool, 0, false, m->side);
-        if (st == PSML_OK && cudaEventRecord(m->ev_join, m->side) != cudaSuccess)
-            st = fail(PSML_ERR_CUDA, "graph join record failed");
+        static int after = -1;
+        if (after < 0) {
+            const char *e = getenv("PSML_DEAL_AFTER");
+            after = e ? std::max(0, atoi(e)) : 1;   // after the step-start open (tools/gpu71.sh)
+        }
+        m->deal_after = after;
+        m->deal_stage = 0;
+        if (st == PSML_OK && after == 0) {
+            st = deal_pool(m, 1 - pool, 0, false, m->side, deal_s2(m));
+            if (st == PSML_OK && cudaEventRecord(m->ev_join, m->side) != cudaSuccess)
+                st = fail(PSML_ERR_CUDA, "graph join record failed");
+        } else {
+            m->deal_pending_pool = 1 - pool;   // forked from the online chain (deal_fork_point)
+        }
     } else if (flags & 1) {
         st = deal_pool(m, pool, 0, false, s);
     }
     m->pool = pool;
     if (st == PSML_OK) st = forward_backward(m, X, Y, on);
+    if (st == PSML_OK) st = deal_fork_point(m, on, true);   // not forked yet: fork here
+    m->deal_pending_pool = -1;
     if (st == PSML_OK && (flags & 2)) {
         m->grads_ready = true;
         st = psml_train_apply_update(m, 0, (psml_stream)on);
