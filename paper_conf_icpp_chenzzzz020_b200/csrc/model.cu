@@ -140,6 +140,8 @@ struct psml_model_s {
     cudaStream_t hi = nullptr;         // online phase inside the pipelined graph (highest priority)
     cudaEvent_t ev_hi = nullptr;
     cudaEvent_t ev_late = nullptr;
+    cudaStream_t gw = nullptr;         // weight-gradient branch of the backward pass (highest priority)
+    cudaEvent_t ev_gw = nullptr, ev_gwj = nullptr;
     cudaStream_t side2 = nullptr;      // second dealer branch (AND / daBit / Hadamard PRG streams)
     cudaEvent_t ev_d2 = nullptr, ev_d2j = nullptr;     // late fork point of the dealer branch (PSML_DEAL_AFTER)
     int deal_pending_pool = -1;        // capture in progress: dealer branch not forked yet
@@ -700,6 +702,15 @@ static psml_status deal_fork_point(psml_model_s *m, cudaStream_t s, bool force =
 }
 
 
+static bool gradw_branch() {
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("PSML_GRADW_BRANCH");
+        v = (e && e[0] == '0') ? 0 : 1;
+    }
+    return v == 1;
+}
+
 static psml_status fused_forward_backward(psml_model_s *m, const T *const X[2], const T *const Y[2], cudaStream_t s) {
     const int F = m->ctx->ring.frac_bits;
     const int nl = m->nl;
@@ -817,13 +828,25 @@ static psml_status fused_forward_backward(psml_model_s *m, const T *const X[2], 
         }
     }
     // 3. backward: gradW_l and gradin_l in one launch, then the backprop Hadamard opens delta_{l-1}
+    //    With PSML_GRADW_BRANCH (default on), gradW_l for l > 0 runs on a second stream as soon as
+    //    delta_l is open, beside the chain gradin_l -> Hadamard -> ... that carries the backward
+    //    dependency (the paper's inter-layer pipeline, Fig. 6, as stream overlap);
+    //    the branch joins before the update.
+    const bool branch = gradw_branch() && nl > 1;
     T *g[2];
     for (int l = nl - 1; l >= 0; --l) {
         gradp(m, l, g);
         SegArgs<T> jobs[2];
         jobs[0] = seg(l, OP_GRADW, g[0], g[1], 0);
         if (l > 0) jobs[1] = seg(l, OP_GRADIN, m->tmp.p[0], m->tmp.p[1], F);
-        PSML_TRY(launch_seg_group<T>(jobs, l > 0 ? 2 : 1, s, m->ctx->sm_count));
+        if (branch && l > 0) {
+            PSML_CUDA_TRY(cudaEventRecord(m->ev_gw, s));
+            PSML_CUDA_TRY(cudaStreamWaitEvent(m->gw, m->ev_gw, 0));
+            PSML_TRY(launch_seg_group<T>(&jobs[0], 1, m->gw, m->ctx->sm_count));
+            PSML_TRY(launch_seg_group<T>(&jobs[1], 1, s, m->ctx->sm_count));
+        } else {
+            PSML_TRY(launch_seg_group<T>(jobs, l > 0 ? 2 : 1, s, m->ctx->sm_count));
+        }
         PSML_TRY(deal_fork_point(m, s));
         if (l > 0) {
             DealItem *h = find_item(m, l - 1, OP_HADAMARD, 1);
@@ -842,6 +865,10 @@ static psml_status fused_forward_backward(psml_model_s *m, const T *const X[2], 
             PSML_CUDA_TRY(launch_pdl(had_fused_kernel<T>, dim3(ew_grid(hf.n)), dim3(EW_THREADS), s, hf));
             PSML_LAUNCH_CHECK();
         }
+    }
+    if (branch) {
+        PSML_CUDA_TRY(cudaEventRecord(m->ev_gwj, m->gw));
+        PSML_CUDA_TRY(cudaStreamWaitEvent(s, m->ev_gwj, 0));
     }
     return PSML_OK;
 }
@@ -1190,12 +1217,15 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
         PSML_CUDA_TRY(cudaStreamCreateWithPriority(&m->side, cudaStreamNonBlocking, lo));
         PSML_CUDA_TRY(cudaStreamCreateWithPriority(&m->side2, cudaStreamNonBlocking, lo));
         PSML_CUDA_TRY(cudaStreamCreateWithPriority(&m->hi, cudaStreamNonBlocking, hi));
+        PSML_CUDA_TRY(cudaStreamCreateWithPriority(&m->gw, cudaStreamNonBlocking, hi));
         PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_hi, cudaEventDisableTiming));
     }
     PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_fork, cudaEventDisableTiming));
     PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_join, cudaEventDisableTiming));
     PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_late, cudaEventDisableTiming));
     PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_d2, cudaEventDisableTiming));
+    PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_gw, cudaEventDisableTiming));
+    PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_gwj, cudaEventDisableTiming));
     PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_d2j, cudaEventDisableTiming));
     {
         T *sd = nullptr;
@@ -1222,6 +1252,9 @@ psml_status psml_model_destroy(psml_model model) {
     if (model->ev_d2) cudaEventDestroy(model->ev_d2);
     if (model->ev_d2j) cudaEventDestroy(model->ev_d2j);
     if (model->side2) cudaStreamDestroy(model->side2);
+    if (model->gw) cudaStreamDestroy(model->gw);
+    if (model->ev_gw) cudaEventDestroy(model->ev_gw);
+    if (model->ev_gwj) cudaEventDestroy(model->ev_gwj);
     for (void *p : model->allocs) cudaFree(p);
     delete model;
     return PSML_OK;
