@@ -176,8 +176,13 @@ def bench_ours(args):
         X, Y = synth.batch(TASK, s, BATCH, pair=rank, n_pairs=world)
         Xs.append(torch.from_numpy(X).to(dev))
         Ys.append(torch.from_numpy(Y).to(dev))
-    Xh = [x.cpu().pin_memory() for x in Xs]
-    Yh = [y.cpu().pin_memory() for y in Ys]
+    # e2e leg: the client's own form of the same batches -- 8-bit pixels and (one-hot tasks)
+    # class indices -- in pinned host memory; they share bit-identically to the float64 batches
+    Xh, Yh = [], []
+    for s in range(nb):
+        q, y = synth.batch_u8(TASK, s, BATCH, pair=rank, n_pairs=world)
+        Xh.append(torch.from_numpy(q).pin_memory())
+        Yh.append(torch.from_numpy(np.ascontiguousarray(y)).pin_memory())
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream()
 
@@ -264,7 +269,7 @@ def bench_ours(args):
     t_on = max_over_ranks(sum(a.elapsed_time(b) for a, b in evs) / 1e3, world)
 
     # e2e through the public API with host buffers: H2D plaintext batch, full step, D2H yhat
-    h2d = Xh[0].numel() * 8 + Yh[0].numel() * 8
+    h2d = Xh[0].numel() * Xh[0].element_size() + Yh[0].numel() * Yh[0].element_size()
     out_host = torch.empty((2, BATCH, Ys[0].shape[1]), dtype=torch.uint64).pin_memory()
     d2h = out_host.numel() * 8
 

@@ -111,6 +111,18 @@ psml_status psml_share(psml_ring ring, uint64_t seed, uint64_t stream_id, const 
  * x: n doubles (device).  Bit-identical to the two calls. */
 psml_status psml_encode_share(psml_ring ring, uint64_t seed, uint64_t stream_id, const double *x,
                               int64_t n, void *x0, void *x1, psml_stream stream);
+/* Client encode + share straight from 8-bit pixels (image pixels 0..255):
+ * x = q / den in fp64 (IEEE division), then exactly psml_encode_share.  q: n bytes (device).
+ * Bit-identical to psml_encode_share on the float64 q / den.  den > 0 (255 for 8-bit images). */
+psml_status psml_encode_share_u8(psml_ring ring, uint64_t seed, uint64_t stream_id, const uint8_t *q,
+                                 int64_t n, double den, void *x0, void *x1, psml_stream stream);
+/* Client encode + share of one-hot labels from class indices: Y[r][c] = (cls[r] == c), encoded
+ * (1 -> 2^frac_bits, 0 -> 0) and shared like psml_encode_share on the float64 one-hot matrix
+ * (rows x classes, row-major).  cls: rows bytes (device); a class index >= classes gives an
+ * all-zero row. */
+psml_status psml_encode_share_onehot(psml_ring ring, uint64_t seed, uint64_t stream_id,
+                                     const uint8_t *cls, int64_t rows, int64_t classes, void *x0,
+                                     void *x1, psml_stream stream);
 /* x = x0 + x1 mod 2^l (client-side reconstruction). */
 psml_status psml_reconstruct(psml_ring ring, const void *x0, const void *x1, int64_t n, void *x,
                              psml_stream stream);

@@ -240,6 +240,38 @@ psml_status psml_encode_share(psml_ring ring, uint64_t seed, uint64_t stream_id,
     return PSML_OK;
 }
 
+static psml_status encode_share_u8(psml_ring ring, uint64_t seed, uint64_t stream_id, const uint8_t *q, int64_t n,
+                                   double den, int64_t classes, void *x0, void *x1, psml_stream stream) {
+    PSML_TRY(check_ring(ring));
+    if (n < 0) return fail(PSML_ERR_SHAPE, "n < 0");
+    if (n == 0) return PSML_OK;
+    PSML_TRY(check_ptrs({q, x0, x1}));
+    if (x0 == x1) return fail(PSML_ERR_INVALID, "share outputs must not alias");
+    cudaStream_t s = (cudaStream_t)stream;
+    PrgKey k = make_key(seed, TAG_SH, stream_id);
+    const int64_t nblk = n / (ring.l == 64 ? 8 : 16) + 1;
+    if (ring.l == 64)
+        encode_share_u8_kernel<uint64_t><<<grid_for(nblk, 128), 128, 0, s>>>(k, n, ring.frac_bits, q, den, classes,
+                                                                              (uint64_t *)x0, (uint64_t *)x1);
+    else
+        encode_share_u8_kernel<uint32_t><<<grid_for(nblk, 128), 128, 0, s>>>(k, n, ring.frac_bits, q, den, classes,
+                                                                              (uint32_t *)x0, (uint32_t *)x1);
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
+psml_status psml_encode_share_u8(psml_ring ring, uint64_t seed, uint64_t stream_id, const uint8_t *q, int64_t n,
+                                 double den, void *x0, void *x1, psml_stream stream) {
+    if (!(den > 0.0)) return fail(PSML_ERR_INVALID, "den must be > 0");
+    return encode_share_u8(ring, seed, stream_id, q, n, den, 1, x0, x1, stream);
+}
+
+psml_status psml_encode_share_onehot(psml_ring ring, uint64_t seed, uint64_t stream_id, const uint8_t *cls,
+                                     int64_t rows, int64_t classes, void *x0, void *x1, psml_stream stream) {
+    if (rows < 0 || classes <= 0) return fail(PSML_ERR_SHAPE, "rows < 0 or classes <= 0");
+    return encode_share_u8(ring, seed, stream_id, cls, rows * classes, 0.0, classes, x0, x1, stream);
+}
+
 psml_status psml_reconstruct(psml_ring ring, const void *x0, const void *x1, int64_t n, void *x,
                              psml_stream stream) {
     PSML_TRY(check_ring(ring));

@@ -62,6 +62,32 @@ __global__ void encode_share_kernel(PrgKey key, int64_t n, int f, const double *
     }
 }
 
+// Same, with the plaintext given as bytes: x = q / den (pixels, den = 255) or, for den = 0, the
+// one-hot row of class index q[e / classes] (x = 1 at column q, else 0).
+template <typename T>
+__global__ void encode_share_u8_kernel(PrgKey key, int64_t n, int f, const uint8_t *__restrict__ q, double den,
+                                       int64_t classes, T *__restrict__ out0, T *__restrict__ out1) {
+    constexpr int PB = PerBlock<T>::value;
+    key = live_key(key);
+    const uint64_t last_blk = ((uint64_t)n - 1) / PB;
+    for (uint64_t b = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; b <= last_blk; b += (uint64_t)gridDim.x * blockDim.x) {
+        uint32_t w[16];
+        chacha20_block(key, (uint32_t)b, w);
+#pragma unroll
+        for (int j = 0; j < PB; ++j) {
+            const uint64_t e = b * PB + j;
+            if (e >= (uint64_t)n) continue;
+            const T r = sizeof(T) == 8 ? (T)(((uint64_t)w[2 * j + 1] << 32) | w[2 * j]) : (T)w[j];
+            double x;
+            if (den > 0.0) x = (double)q[e] / den;
+            else x = (int64_t)q[e / (uint64_t)classes] == (int64_t)(e % (uint64_t)classes) ? 1.0 : 0.0;
+            const T v = (T)(unsigned long long)__double2ll_rn(ldexp(x, f));
+            out0[e] = r;
+            out1[e] = v - r;
+        }
+    }
+}
+
 template <typename T>
 __global__ void encode_kernel(const double *__restrict__ x, int64_t n, int f, T *__restrict__ v) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {

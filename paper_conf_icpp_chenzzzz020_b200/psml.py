@@ -66,6 +66,8 @@ _SIGS = {
     "psml_share": (i32, [Ring, u64, u64, vp, i64, vp, vp, vp]),
     "psml_reconstruct": (i32, [Ring, vp, vp, i64, vp, vp]),
     "psml_encode_share": (i32, [Ring, u64, u64, vp, i64, vp, vp, vp]),
+    "psml_encode_share_u8": (i32, [Ring, u64, u64, vp, i64, ctypes.c_double, vp, vp, vp]),
+    "psml_encode_share_onehot": (i32, [Ring, u64, u64, vp, i64, i64, vp, vp, vp]),
     "psml_triplet_gen": (i32, [vp, u64, u64, i64, i64, i64, P2, P2, P2, vp]),
     "psml_hadamard_triplet_gen": (i32, [Ring, u64, u64, i64, P2, P2, P2, vp]),
     "psml_msb_material_words": (i64, [Ring, i64]),
@@ -265,6 +267,28 @@ def encode_share(ring, seed, stream_id, x, out=None, stream=None):
     x0, x1 = out if out is not None else empty_pair(x.shape, ring.l)
     _call("psml_encode_share", ring, seed, stream_id, _ptr(x), x.numel(), _ptr(x0), _ptr(x1),
           _stream(stream))
+    return x0, x1
+
+
+def encode_share_u8(ring, seed, stream_id, q, den=255.0, out=None, stream=None):
+    """encode_share of q / den from bytes (q: uint8 device tensor, e.g. 8-bit pixels)."""
+    if q.dtype != torch.uint8:
+        raise PsmlError("marshal", 1, "encode_share_u8 takes uint8")
+    q = q.contiguous()
+    x0, x1 = out if out is not None else empty_pair(q.shape, ring.l)
+    _call("psml_encode_share_u8", ring, seed, stream_id, _ptr(q), q.numel(), float(den), _ptr(x0), _ptr(x1),
+          _stream(stream))
+    return x0, x1
+
+
+def encode_share_onehot(ring, seed, stream_id, cls, classes, out=None, stream=None):
+    """encode_share of the one-hot (rows x classes) matrix of class indices cls (uint8 device)."""
+    if cls.dtype != torch.uint8:
+        raise PsmlError("marshal", 1, "encode_share_onehot takes uint8 class indices")
+    cls = cls.contiguous()
+    x0, x1 = out if out is not None else empty_pair((cls.numel(), classes), ring.l)
+    _call("psml_encode_share_onehot", ring, seed, stream_id, _ptr(cls), cls.numel(), classes, _ptr(x0),
+          _ptr(x1), _stream(stream))
     return x0, x1
 
 

@@ -52,13 +52,28 @@ class SecureTrainer:
         self.out_dim = self.model.layer_shape(self.model.n_layers - 1)[1]
 
     # --- client side -----------------------------------------------------------------------
-    def share_batch(self, X, Y, step):
-        """Encode + share one minibatch on the GPU (X, Y: float64 tensors, host or device)."""
-        Xs = psml.encode_share(self.ring, SHARE_SEED, call_id(self.pair_id, step, 0, OP_SHARE, 0),
-                               _dev64(X))
-        Ys = psml.encode_share(self.ring, SHARE_SEED, call_id(self.pair_id, step, 0, OP_SHARE, 1),
-                               _dev64(Y))
+    def _client_share(self, X, Y, step, outX=None, outY=None):
+        """Client encode + share of a minibatch into (outX, outY): X float64
+        features, or uint8 pixels (x = q / 255, synth.batch_u8); Y float64 labels, or uint8 class
+        indices of one-hot labels.  Both forms give bit-identical shares."""
+        cx = call_id(self.pair_id, step, 0, OP_SHARE, 0)
+        cy = call_id(self.pair_id, step, 0, OP_SHARE, 1)
+        if torch.is_tensor(X) and X.dtype == torch.uint8:
+            Xs = psml.encode_share_u8(self.ring, SHARE_SEED, cx, X if X.is_cuda else X.cuda(non_blocking=True),
+                                      255.0, out=outX)
+        else:
+            Xs = psml.encode_share(self.ring, SHARE_SEED, cx, _dev64(X), out=outX)
+        if torch.is_tensor(Y) and Y.dtype == torch.uint8:
+            Ys = psml.encode_share_onehot(self.ring, SHARE_SEED, cy, Y if Y.is_cuda else Y.cuda(non_blocking=True),
+                                          self.out_dim, out=outY)
+        else:
+            Ys = psml.encode_share(self.ring, SHARE_SEED, cy, _dev64(Y), out=outY)
         return Xs, Ys
+
+    def share_batch(self, X, Y, step):
+        """Encode + share one minibatch on the GPU (X, Y: float64 tensors, host or device; or the
+        uint8 pixel / class-index form, see _client_share)."""
+        return self._client_share(X, Y, step)
 
     # --- steps --------------------------------------------------------------------------------
     def capture(self, with_update=True, pipelined=True):
@@ -85,10 +100,7 @@ class SecureTrainer:
 
     def graph_step(self, X, Y, step):
         """Client encode + share into the captured buffers, then replay the captured step."""
-        psml.encode_share(self.ring, SHARE_SEED, call_id(self.pair_id, step, 0, OP_SHARE, 0), _dev64(X),
-                          out=self.Xbuf)
-        psml.encode_share(self.ring, SHARE_SEED, call_id(self.pair_id, step, 0, OP_SHARE, 1), _dev64(Y),
-                          out=self.Ybuf)
+        self._client_share(X, Y, step, outX=self.Xbuf, outY=self.Ybuf)
         if self.pipelined and self._next_dealt != step:
             self.model.deal(step)          # prime the pipeline (first step or a jump in step ids)
         self.model.step_graph(step)

@@ -4,9 +4,12 @@ This module holds NONE of the method's arithmetic (no encoding, sharing, ring or
 step): it only produces float64 plaintext data, labels and initial weights with the shapes and
 value distributions of the paper's workloads:
 
-  * MNIST-shaped rows (28x28 pixels 0..255): 784 features in [0, 1], about 81%
-    exact zeros, non-zeros U(0, 1] (MNIST's ~19% ink density), scaled by 1/255 semantics.
-  * CIFAR-10-shaped rows (3x32x32): 3072 dense U(0, 1) features.
+  * MNIST-shaped rows (28x28 pixels 0..255): 784 8-bit pixels k, about 81%
+    zeros, non-zeros uniform on 1..255 (MNIST's ~19% ink density); features x = k / 255.
+  * CIFAR-10-shaped rows (3x32x32): 3072 dense 8-bit pixels uniform on 0..255,
+    x = k / 255.
+  * the pixel bytes themselves (`batch_u8`): what a client holding the images sends; the float64
+    features are exactly k / 255.0 (IEEE division), so both forms encode to the same ring words.
   * labels from fixed random teachers (linear, thresholded linear, 784-128-128-10 ReLU MLP,
     5x5/16-channel conv net), one-hot for the 10-class tasks.
 
@@ -30,24 +33,30 @@ CIFAR_FEATURES = 3 * 32 * 32
 _KIND = {"mnist": 1, "cifar": 2}
 
 
-def _block_rows(kind, b, seed):
+def _block_pixels(kind, b, seed):
     rng = np.random.default_rng([seed, _KIND[kind], b])
     if kind == "mnist":
         x = rng.random((BLOCK, MNIST_FEATURES))
         keep = rng.random((BLOCK, MNIST_FEATURES)) < 0.19
-        return np.where(keep, 1.0 - x, 0.0)                 # non-zeros in (0, 1]
-    return rng.random((BLOCK, CIFAR_FEATURES))
+        k = np.minimum(np.floor(x * 255.0), 254.0).astype(np.uint8) + 1   # 1..255
+        return np.where(keep, k, 0).astype(np.uint8)
+    return np.minimum(np.floor(rng.random((BLOCK, CIFAR_FEATURES)) * 256.0), 255.0).astype(np.uint8)
+
+
+def pixels(kind, start, count, seed=DATA_SEED):
+    """8-bit pixels of rows [start, start+count) of the synthetic dataset `kind`."""
+    if count <= 0:
+        width = MNIST_FEATURES if kind == "mnist" else CIFAR_FEATURES
+        return np.zeros((0, width), dtype=np.uint8)
+    b0, b1 = start // BLOCK, (start + count - 1) // BLOCK
+    blocks = np.concatenate([_block_pixels(kind, b, seed) for b in range(b0, b1 + 1)], axis=0)
+    off = start - b0 * BLOCK
+    return blocks[off:off + count]
 
 
 def rows(kind, start, count, seed=DATA_SEED):
-    """Rows [start, start+count) of the synthetic dataset `kind` ('mnist' | 'cifar')."""
-    if count <= 0:
-        width = MNIST_FEATURES if kind == "mnist" else CIFAR_FEATURES
-        return np.zeros((0, width))
-    b0, b1 = start // BLOCK, (start + count - 1) // BLOCK
-    blocks = np.concatenate([_block_rows(kind, b, seed) for b in range(b0, b1 + 1)], axis=0)
-    off = start - b0 * BLOCK
-    return blocks[off:off + count]
+    """Rows [start, start+count) of the synthetic dataset `kind` ('mnist' | 'cifar'): k / 255."""
+    return pixels(kind, start, count, seed).astype(np.float64) / 255.0
 
 
 # ---------------------------------------------------------------------------------------------
@@ -124,6 +133,19 @@ def batch(task, step, batch_size=BLOCK, pair=0, n_pairs=1, seed=DATA_SEED):
     start = ((step * n_pairs + pair) * batch_size) % (TASK_ROWS[kind] - batch_size + 1)
     X = rows(kind, start, batch_size, seed)
     return X, labels(task, X)
+
+
+def batch_u8(task, step, batch_size=BLOCK, pair=0, n_pairs=1, seed=DATA_SEED):
+    """The same minibatch as `batch` in the client's compact form: (pixels uint8, labels), labels
+    as uint8 class indices for the one-hot tasks (mlp, cnn), else the float64 labels of `batch`.
+    batch() == (pixels / 255.0, one_hot(classes)) exactly."""
+    kind = TASK_DATA[task]
+    start = ((step * n_pairs + pair) * batch_size) % (TASK_ROWS[kind] - batch_size + 1)
+    q = pixels(kind, start, batch_size, seed)
+    Y = labels(task, q.astype(np.float64) / 255.0)
+    if task in ("mlp", "cnn"):
+        return q, np.argmax(Y, axis=1).astype(np.uint8)
+    return q, Y
 
 
 def init_weights(task, dims=None, seed=INIT_SEED):

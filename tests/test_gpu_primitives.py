@@ -70,6 +70,29 @@ def test_encode_decode_share_reconstruct(P, orc, l):
 
 
 @pytest.mark.parametrize("l", [64, 32])
+def test_encode_share_from_pixels_and_class_indices(P, orc, l):
+    """psml_encode_share_u8 (x = q / 255 from 8-bit pixels) and psml_encode_share_onehot (one-hot
+    labels from class indices) equal the oracle's encode + share of the float64 batch, on the
+    synthetic MNIST/CIFAR batches and on ragged sizes, every pixel value 0..255 included."""
+    import synth
+    ring = P.Ring(l, 13)
+    for task in ("mlp", "cnn"):
+        X, Y = synth.batch(task, 5)
+        q, cls = synth.batch_u8(task, 5)
+        x0, x1 = P.encode_share_u8(ring, SEED + 1, 44, torch.from_numpy(q).cuda())
+        w0, w1 = orc.share(orc.encode(X.reshape(-1), l, 13), SEED + 1, 44, l)
+        assert np.array_equal(to_np(x0).reshape(-1), w0) and np.array_equal(to_np(x1).reshape(-1), w1), task
+        y0, y1 = P.encode_share_onehot(ring, SEED + 1, 45, torch.from_numpy(cls).cuda(), 10)
+        v0, v1 = orc.share(orc.encode(Y.reshape(-1), l, 13), SEED + 1, 45, l)
+        assert np.array_equal(to_np(y0).reshape(-1), v0) and np.array_equal(to_np(y1).reshape(-1), v1), task
+    q = np.arange(256, dtype=np.uint8)
+    for n in (1, 9, 256):
+        x0, x1 = P.encode_share_u8(ring, SEED + 1, 46, torch.from_numpy(q[:n]).cuda())
+        w0, w1 = orc.share(orc.encode(q[:n].astype(np.float64) / 255.0, l, 13), SEED + 1, 46, l)
+        assert np.array_equal(to_np(x0), w0) and np.array_equal(to_np(x1), w1), n
+
+
+@pytest.mark.parametrize("l", [64, 32])
 def test_truncate(P, orc, l):
     ring = P.Ring(l, 13)
     x = _rand(orc, l, 10007, 1)

@@ -99,3 +99,19 @@ def test_diagnostics_zero_failures_and_checker_pinned():
         assert P.DIAG["trunc_fail"] == 0 and P.DIAG["trunc_checked"] == 2
     finally:
         P.diag_reset(False)
+
+
+def test_synthetic_batches_are_8bit_pixels():
+    """Input recipe: features are 8-bit pixels / 255,
+    ~19% non-zero for MNIST-shaped rows, dense for CIFAR-shaped; batch_u8 is the same batch in
+    the client's byte form (pixels, class indices of the one-hot labels)."""
+    for task in ("mlp", "cnn", "linreg", "logreg"):
+        X, Y = synth.batch(task, 7)
+        q, y = synth.batch_u8(task, 7)
+        assert q.dtype == np.uint8 and np.array_equal(X, q.astype(np.float64) / 255.0)
+        if task in ("mlp", "cnn"):
+            assert y.dtype == np.uint8 and np.array_equal(Y, np.eye(10)[y])
+        else:
+            assert np.array_equal(Y, y)
+    X, _ = synth.batch("mlp", 0)
+    assert 0.17 < (X > 0).mean() < 0.21 and X.max() == 1.0 and X[X > 0].min() >= 1 / 255
