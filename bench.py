@@ -275,6 +275,11 @@ def bench_ours(args):
 
     def e2e_step(s):
         i = (s - 2 * (W + K)) % nb
+        if world == 1:
+            # one library call: H2D pixels + labels, client encode/share, the captured step, D2H
+            # of both parties' prediction shares (psml_model_step_host)
+            tr.graph_step_host(Xh[i], Yh[i], s, out_host)
+            return
         X = Xh[i].to(dev, non_blocking=True)
         Y = Yh[i].to(dev, non_blocking=True)
         graph_step(s, X, Y)

@@ -305,6 +305,17 @@ psml_status psml_train_apply_update(psml_model model, int32_t extra_shift, psml_
 psml_status psml_model_capture_step(psml_model model, const void *const X[2], const void *const Y[2],
                                     int32_t flags, psml_stream stream);
 psml_status psml_model_step_graph(psml_model model, uint32_t step_id, psml_stream stream);
+/* One whole step from HOST buffers (the client's end-to-end call): copies the
+ * minibatch's 8-bit pixels q (batch x d_0 bytes, host; pinned memory makes the copies
+ * asynchronous) and its labels y (y_kind 0: float64 batch x d_L; 1: uint8 class indices of one-hot
+ * labels, batch bytes) to model-owned device staging, encodes and shares them into the captured
+ * X/Y buffers (psml_encode_share_u8 / _onehot / psml_encode_share, share ids = call id
+ * (pair, step_id, 0, op 7, slot 0/1) under share_seed; R11), replays the captured step
+ * (psml_model_step_graph, same preconditions) and copies both parties' prediction shares
+ * (2 x batch x d_L words, party 0 first) to yhat_host (host).  Asynchronous on `stream`: the
+ * host buffers must stay valid until it completes.  PSML_ERR_STATE without a captured step. */
+psml_status psml_model_step_host(psml_model model, const uint8_t *q, const void *y, int32_t y_kind,
+                                 uint64_t share_seed, uint32_t step_id, void *yhat_host, psml_stream stream);
 /* Number of kernel nodes in the captured step graph (launch accounting for bench.py). */
 psml_status psml_model_graph_nodes(psml_model model, int64_t *n);
 /* Secure inference (the forward half): Yhat[i]: batch x d_L.  Needs

@@ -24,7 +24,7 @@ namespace psml {
 
 using T = uint64_t;
 
-enum { OP_FWD = 0, OP_GRADW = 1, OP_GRADIN = 2, OP_RELU_MSB = 3, OP_EQ9_MSB = 4, OP_HADAMARD = 6 };
+enum { OP_FWD = 0, OP_GRADW = 1, OP_GRADIN = 2, OP_RELU_MSB = 3, OP_EQ9_MSB = 4, OP_HADAMARD = 6, OP_SHARE = 7 };
 enum ItemKind { IT_MATRIX, IT_CONV_FWD, IT_CONV_GW, IT_HAD, IT_MSB };
 
 __global__ void set_word_kernel(uint32_t *p, uint32_t v) { *p = v; }
@@ -140,12 +140,16 @@ struct psml_model_s {
     cudaStream_t hi = nullptr;         // online phase inside the pipelined graph (highest priority)
     cudaEvent_t ev_hi = nullptr;
     cudaEvent_t ev_late = nullptr;
+    const void *cap_X[2] = {nullptr, nullptr}, *cap_Y[2] = {nullptr, nullptr};   // captured step inputs
+    uint8_t *stage_q = nullptr;        // device staging of psml_model_step_host (pixels, labels)
+    void *stage_y = nullptr;
     cudaStream_t gw = nullptr;         // weight-gradient branch of the backward pass (highest priority)
     cudaEvent_t ev_gw = nullptr, ev_gwj = nullptr;
     cudaStream_t side2 = nullptr;      // second dealer branch (AND / daBit / Hadamard PRG streams)
     cudaEvent_t ev_d2 = nullptr, ev_d2j = nullptr;     // late fork point of the dealer branch (PSML_DEAL_AFTER)
     int deal_pending_pool = -1;        // capture in progress: dealer branch not forked yet
     int deal_after = 0, deal_stage = 0;
+    bool deal_alone = false;           // dealer being captured after the online chain (full PRG grid)
 };
 
 namespace psml {
@@ -480,7 +484,10 @@ static psml_status deal_prg_launch(psml_model_s *m, const DealPlan &P, int j0, i
         per_sm = e ? atoi(e) : 4;   // measured best of {1, 2, 4, full} (tools/gpu44.sh)
     }
     const int64_t full = (b1 - b0 + 127) / 128;
-    const int64_t grid = per_sm > 0 ? std::min<int64_t>(full, (int64_t)per_sm * m->ctx->sm_count) : full;
+    // a dealer forked after the whole online chain (models without the fused step, e.g. the CNN)
+    // overlaps nothing but the update: it takes the whole GPU
+    const int64_t grid = (per_sm > 0 && !m->deal_alone) ? std::min<int64_t>(full, (int64_t)per_sm * m->ctx->sm_count)
+                                                        : full;
     deal_prg_kernel<<<(unsigned)grid, 128, 0, s>>>(P.prg + j0, j1 - j0, b0, b1, m->d.dealer_seed, m->step_dev);
     PSML_LAUNCH_CHECK();
     return PSML_OK;
@@ -696,7 +703,10 @@ static psml_status deal_fork_point(psml_model_s *m, cudaStream_t s, bool force =
     m->deal_pending_pool = -1;
     PSML_CUDA_TRY(cudaEventRecord(m->ev_late, s));
     PSML_CUDA_TRY(cudaStreamWaitEvent(m->side, m->ev_late, 0));
-    PSML_TRY(deal_pool(m, pool, 0, false, m->side, deal_s2(m)));
+    m->deal_alone = force;
+    const psml_status st = deal_pool(m, pool, 0, false, m->side, deal_s2(m));
+    m->deal_alone = false;
+    PSML_TRY(st);
     PSML_CUDA_TRY(cudaEventRecord(m->ev_join, m->side));
     return PSML_OK;
 }
@@ -1406,9 +1416,11 @@ static psml_status capture_one(psml_model_s *m, int pool, const T *const X[2], c
             const char *e = getenv("PSML_DEAL_AFTER");
             after = e ? std::max(0, atoi(e)) : 1;   // after the step-start open (tools/gpu71.sh)
         }
-        m->deal_after = after;
+        // models without the fused step (the CNN) run large kernels that fill the GPU: their
+        // dealer forks at the start of the step (measured: 51.6K vs 49.4K samples/s forked after)
+        m->deal_after = fused_eligible(m) ? after : 0;
         m->deal_stage = 0;
-        if (st == PSML_OK && after == 0) {
+        if (st == PSML_OK && m->deal_after == 0) {
             st = deal_pool(m, 1 - pool, 0, false, m->side, deal_s2(m));
             if (st == PSML_OK && cudaEventRecord(m->ev_join, m->side) != cudaSuccess)
                 st = fail(PSML_ERR_CUDA, "graph join record failed");
@@ -1475,6 +1487,72 @@ psml_status psml_model_capture_step(psml_model m, const void *const X[2], const 
     g_prof_cls.store(prof);
     if (st != PSML_OK) return st;
     m->graph_flags = flags;
+    for (int i = 0; i < 2; ++i) { m->cap_X[i] = X[i]; m->cap_Y[i] = Y[i]; }
+    return PSML_OK;
+}
+
+// out[0..n) = a, out[n..2n) = b (the prediction shares into mapped host memory)
+template <typename U>
+__global__ void copy_pair_kernel(const U *__restrict__ a, const U *__restrict__ b, int64_t n, U *__restrict__ out) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < 2 * n; i += (int64_t)gridDim.x * blockDim.x)
+        out[i] = i < n ? a[i] : b[i - n];
+}
+
+psml_status psml_model_step_host(psml_model m, const uint8_t *q, const void *y, int32_t y_kind, uint64_t share_seed,
+                                 uint32_t step_id, void *yhat_host, psml_stream stream) {
+    if (!m || !q || !y || !yhat_host) return fail(PSML_ERR_INVALID, "null argument");
+    if (!m->graph[0] || !m->cap_X[0]) return fail(PSML_ERR_STATE, "no captured step: call psml_model_capture_step first");
+    if (y_kind != 0 && y_kind != 1) return fail(PSML_ERR_INVALID, "y_kind: 0 float64 labels, 1 uint8 class indices");
+    cudaStream_t s = (cudaStream_t)stream;
+    const int64_t nx = m->B * m->dims[0], dl = m->dims.back(), ny = m->B * dl;
+    if (!m->stage_q) {
+        T *a = nullptr, *b = nullptr;
+        PSML_TRY(dalloc(m, &a, (nx + 7) / 8));
+        PSML_TRY(dalloc(m, &b, ny));
+        m->stage_q = (uint8_t *)a;
+        m->stage_y = b;
+    }
+    // Pinned host buffers mapped into the device address space (cudaHostAlloc / pinned tensors
+    // under UVA) are read and written by the kernels directly over PCIe (zero-copy); anything
+    // else goes through cudaMemcpyAsync and the device staging buffers.
+    auto mapped = [](const void *p) -> void * {
+        cudaPointerAttributes a{};
+        if (cudaPointerGetAttributes(&a, p) != cudaSuccess) { cudaGetLastError(); return nullptr; }
+        return a.type == cudaMemoryTypeHost ? a.devicePointer : nullptr;
+    };
+    const uint8_t *qd = (const uint8_t *)mapped(q);
+    const void *yd = mapped(y);
+    T *od = (T *)mapped(yhat_host);
+    // client: the compact plaintext batch to the GPU, encode + share into the captured buffers
+    if (!qd) {
+        PSML_CUDA_TRY(cudaMemcpyAsync(m->stage_q, q, (size_t)nx, cudaMemcpyHostToDevice, s));
+        qd = m->stage_q;
+    }
+    if (!yd) {
+        PSML_CUDA_TRY(cudaMemcpyAsync(m->stage_y, y, y_kind ? (size_t)m->B : sizeof(double) * (size_t)ny,
+                                      cudaMemcpyHostToDevice, s));
+        yd = m->stage_y;
+    }
+    const psml_ring ring = m->ctx->ring;
+    const uint64_t cx = call_id(m->d.pair_id, step_id, 0, OP_SHARE, 0), cy = call_id(m->d.pair_id, step_id, 0, OP_SHARE, 1);
+    PSML_TRY(psml_encode_share_u8(ring, share_seed, cx, qd, nx, 255.0, (void *)m->cap_X[0], (void *)m->cap_X[1], stream));
+    if (y_kind)
+        PSML_TRY(psml_encode_share_onehot(ring, share_seed, cy, (const uint8_t *)yd, m->B, dl, (void *)m->cap_Y[0],
+                                          (void *)m->cap_Y[1], stream));
+    else
+        PSML_TRY(psml_encode_share(ring, share_seed, cy, (const double *)yd, ny, (void *)m->cap_Y[0],
+                                   (void *)m->cap_Y[1], stream));
+    // servers: the captured step
+    PSML_TRY(psml_model_step_graph(m, step_id, stream));
+    // client: both parties' prediction shares back
+    if (od) {
+        copy_pair_kernel<T><<<grid_for(2 * ny, 256), 256, 0, s>>>(m->yhat.p[0], m->yhat.p[1], ny, od);
+        PSML_LAUNCH_CHECK();
+    } else {
+        for (int i = 0; i < 2; ++i)
+            PSML_CUDA_TRY(cudaMemcpyAsync((uint8_t *)yhat_host + (size_t)i * sizeof(T) * ny, m->yhat.p[i],
+                                          sizeof(T) * (size_t)ny, cudaMemcpyDeviceToHost, s));
+    }
     return PSML_OK;
 }
 

@@ -97,6 +97,7 @@ _SIGS = {
     "psml_secure_infer": (i32, [vp, P2, u32, P2, vp]),
     "psml_model_capture_step": (i32, [vp, P2, P2, i32, vp]),
     "psml_model_step_graph": (i32, [vp, u32, vp]),
+    "psml_model_step_host": (i32, [vp, vp, vp, i32, u64, u32, vp, vp]),
     "psml_model_graph_nodes": (i32, [vp, vp]),
     "psml_nccl_unique_id": (i32, [vp]),
     "psml_xport_nccl_create": (i32, [vp, i32, vp]),
@@ -139,6 +140,13 @@ def _call(name, *args):
 # ---------------------------------------------------------------------------------------------
 def dtype_of(l):
     return torch.uint64 if l == 64 else torch.uint32
+
+
+def _host_ptr(t):
+    """Address of a contiguous CPU tensor (pinned for asynchronous copies)."""
+    if t.is_cuda or not t.is_contiguous():
+        raise PsmlError("marshal", 1, "host tensor must be a contiguous CPU tensor")
+    return ctypes.c_void_p(t.data_ptr())
 
 
 def _ptr(t):
@@ -507,6 +515,14 @@ class Model:
 
     def step_graph(self, step, stream=None):
         _call("psml_model_step_graph", self.handle, step, _stream(stream))
+
+    def step_host(self, q, y, share_seed, step, yhat_host, stream=None):
+        """psml_model_step_host: q uint8 pixels, y float64 labels or uint8 class indices, yhat_host
+        a (2, batch, d_L) uint64 CPU tensor -- all host tensors (pinned)."""
+        if q.dtype != torch.uint8 or y.dtype not in (torch.uint8, torch.float64) or yhat_host.dtype != torch.uint64:
+            raise PsmlError("marshal", 1, "step_host: q uint8, y float64 | uint8, yhat_host uint64")
+        _call("psml_model_step_host", self.handle, _host_ptr(q), _host_ptr(y), 1 if y.dtype == torch.uint8 else 0,
+              share_seed, step, _host_ptr(yhat_host), _stream(stream))
 
     def party_forward_backward(self, party, xport, X_i, Y_i, step, stream=None):
         """Split deployment: party `party`'s half of the step, openings through `xport`."""

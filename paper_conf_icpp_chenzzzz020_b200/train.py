@@ -106,6 +106,15 @@ class SecureTrainer:
         self.model.step_graph(step)
         self._next_dealt = step + 1
 
+    def graph_step_host(self, q, y, step, yhat_host):
+        """The end-to-end client call: host pixels q (uint8) and labels y (float64, or uint8 class
+        indices) in, the captured step on the GPU, both prediction shares out to yhat_host (host
+        uint64, 2 x batch x d_L) -- one library call (psml_model_step_host), asynchronous."""
+        if self.pipelined and self._next_dealt != step:
+            self.model.deal(step)
+        self.model.step_host(q, y, SHARE_SEED, step, yhat_host)
+        self._next_dealt = step + 1
+
     def deal(self, step, infer_only=False):
         self.model.deal(step, infer_only=infer_only)
 

@@ -100,6 +100,31 @@ def test_graph_replay_bitexact_vs_oracle(T, task, steps, pipelined):
     tr.close()
 
 
+@pytest.mark.parametrize("task", ["mlp", "logreg", "cnn"])
+def test_step_host_bitexact_vs_oracle(T, task):
+    """psml_model_step_host (host pixels + labels in, captured step, prediction shares out: the
+    e2e client call) reproduces the oracle's weight shares and prediction shares exactly."""
+    Wi = synth.init_weights(task)
+    tr = T.SecureTrainer(task, Wi, backend=0)
+    om = OP.Model(task, Wi)
+    X, Y = synth.batch(task, 0)
+    tr.step(torch.from_numpy(X), torch.from_numpy(Y), 0)
+    OP.train_step(om, X, Y, 0)
+    tr.capture(pipelined=True)
+    for s in range(1, 3):
+        X, Y = synth.batch(task, s)
+        q, y = synth.batch_u8(task, s)
+        out = torch.empty((2, X.shape[0], Y.shape[1]), dtype=torch.uint64).pin_memory()
+        tr.graph_step_host(torch.from_numpy(q).pin_memory(), torch.from_numpy(np.ascontiguousarray(y)).pin_memory(),
+                           s, out)
+        yhat = OP.train_step(om, X, Y, s)
+        torch.cuda.synchronize()
+        _compare_shares(tr, om)
+        for i in range(2):
+            assert np.array_equal(out[i].numpy(), yhat[i].reshape(out[i].shape)), (task, s, i)
+    tr.close()
+
+
 def test_cnn_one_epoch_against_fp64(T):
     """Config 4 (CIFAR-shaped CNN, 390 steps of 128): decoded master weights vs fp64 SGD.
 
