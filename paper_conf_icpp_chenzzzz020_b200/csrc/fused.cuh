@@ -115,9 +115,16 @@ struct HadFused {
 template <typename T>
 __global__ void __launch_bounds__(256) had_fused_kernel(const __grid_constant__ HadFused<T> h) {
     pdl_trigger();
+    // the Hadamard triplet of the first element is dealer material (complete before any PDL
+    // predecessor started, see msb_chain_pair_kernel): load it before griddepcontrol.wait
+    const int64_t i0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    T pu0 = 0, pu1 = 0, pv0 = 0, pv1 = 0;
+    if (i0 < h.n) { pu0 = h.U[0][i0]; pu1 = h.U[1][i0]; pv0 = h.V[0][i0]; pv1 = h.V[1][i0]; }
     pdl_wait();
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < h.n; i += (int64_t)gridDim.x * blockDim.x) {
-        const T u0 = h.U[0][i], u1 = h.U[1][i], v0 = h.V[0][i], v1 = h.V[1][i];
+    for (int64_t i = i0; i < h.n; i += (int64_t)gridDim.x * blockDim.x) {
+        const bool first = i == i0;
+        const T u0 = first ? pu0 : h.U[0][i], u1 = first ? pu1 : h.U[1][i];
+        const T v0 = first ? pv0 : h.V[0][i], v1 = first ? pv1 : h.V[1][i];
         const T E = (T)(h.a[0][i] - u0) + (T)(h.a[1][i] - u1);
         const T F = (T)(h.b[0][i] - v0) + (T)(h.b[1][i] - v1);
         const T c0 = E * v0 + u0 * F + h.Z[0][i];

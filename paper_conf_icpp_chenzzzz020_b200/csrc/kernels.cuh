@@ -564,7 +564,6 @@ __device__ __forceinline__ T peer_of(T v) {
 template <typename T, int MODE>
 __global__ void __launch_bounds__(256) msb_chain_pair_kernel(MsbArgs<T> a, ChainOut<T> o) {
     pdl_trigger();
-    pdl_wait();
     constexpr int l = 8 * (int)sizeof(T);
     constexpr int L = sizeof(T) == 8 ? 6 : 5;
     const int lane = threadIdx.x & 31;
@@ -587,6 +586,10 @@ __global__ void __launch_bounds__(256) msb_chain_pair_kernel(MsbArgs<T> a, Chain
     const T *mat = p ? a.mat.p[1] : a.mat.p[0];
     // Every load of the chain is data-independent: issue them all up front (one memory round trip
     // instead of one per protocol round -- the rounds' message stores would otherwise order them).
+    // The dealer material (AND triplets, daBit, Hadamard triplet, the consumers' masks) was
+    // written by a kernel that completed before any PDL predecessor of this one could start (the
+    // previous graph's dealer, or a dealer launch without early trigger), so it is loaded BEFORE
+    // griddepcontrol.wait, overlapping the predecessor's tail; only x depends on the predecessor.
     T mt[2 * L][3];
 #pragma unroll
     for (int t = 0; t < 2 * L; ++t)
@@ -594,12 +597,8 @@ __global__ void __launch_bounds__(256) msb_chain_pair_kernel(MsbArgs<T> a, Chain
         for (int w = 0; w < 3; ++w) mt[t][w] = mat[((int64_t)t * 3 + w) * n + e];
     const int64_t off = (int64_t)2 * L * 3 * n;
     const T rB = mat[off + e], rA = mat[off + n + e];
-    const T *xin = p ? a.x.p[1] : a.x.p[0];
-    const T half = p == 0 ? a.half : (T)0;
-    const T x = a.mode == 0 ? xin[e] : (e < (n >> 1) ? xin[e] + half : xin[e - (n >> 1)] - half);
     T hu = 0, hv = 0, hz = 0, ysub = 0;
     if (MODE != 0) { hu = SEL(o.U)[e]; hv = SEL(o.V)[e]; hz = SEL(o.Z)[e]; }
-    if (MODE == 2 && !second && SEL(o.Ysub)) ysub = SEL(o.Ysub)[e];
     T emk[2] = {0, 0};
     int64_t edi[2] = {0, 0};
 #pragma unroll
@@ -608,6 +607,11 @@ __global__ void __launch_bounds__(256) msb_chain_pair_kernel(MsbArgs<T> a, Chain
             edi[q] = emit_index(o.em.e[q], e);
             emk[q] = o.em.e[q].M[p][edi[q]];
         }
+    pdl_wait();
+    const T *xin = p ? a.x.p[1] : a.x.p[0];
+    const T half = p == 0 ? a.half : (T)0;
+    const T x = a.mode == 0 ? xin[e] : (e < (n >> 1) ? xin[e] + half : xin[e - (n >> 1)] - half);
+    if (MODE == 2 && !second && SEL(o.Ysub)) ysub = SEL(o.Ysub)[e];
     // consumer opens of this lane pair's value v (both parties: v here, the peer's by shuffle)
     auto emit = [&](T v, bool ok) {
 #pragma unroll

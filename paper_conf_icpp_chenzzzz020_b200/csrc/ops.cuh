@@ -71,7 +71,7 @@ psml_status beaver_matmul(const T *const A[2], const T *const B[2], const T *con
             mask_kernel<T><<<dim3((unsigned)std::min<int64_t>(maxt, 148 * 8), 1, (unsigned)count), dim3(32, 8), 0, s>>>(tj);
             PSML_LAUNCH_CHECK();
         }
-        SegArgs<T> sa;
+        SegArgs<T> sa{};
         sa.X[0] = U[0]; sa.X[1] = X1; sa.E = E; sa.F = F;
         for (int p = 0; p < 2; ++p) { sa.V[p] = V[p]; sa.Z[p] = Z[p]; sa.C[p] = C[p]; sa.party[p] = p; }
         sa.M = M; sa.N = N; sa.K = K; sa.trunc = trunc;
