@@ -444,11 +444,12 @@ def measured_peaks():
 
 def committed_traffic(name):
     """DRAM bytes per launch of kernel class `name` from the committed ncu --set full capture
-    (profiles/r01c_traffic.json), or None."""
+    (the newest profiles/r01*_traffic.json, written by tools/traffic.py), or None."""
+    import glob
     try:
-        t = json.load(open(os.path.join(ROOT, "profiles", "r01c_traffic.json")))
+        t = json.load(open(sorted(glob.glob(os.path.join(ROOT, "profiles", "r01*_traffic.json")))[-1]))
         return t[name]["bytes_per_launch_avg"], t["source"]
-    except (OSError, ValueError, KeyError):
+    except (OSError, ValueError, KeyError, IndexError):
         return None, None
 
 

@@ -109,8 +109,6 @@ struct SegArgs {
     int64_t M, N, K;
     int trunc;
     int nparty;        // 1 (split deployment) or 2 (co-resident)
-    int dealer_pre;    // 1: X[0] and V[p] are dealer material complete before any PDL predecessor
-                       //    started (the fused training step): loaded before griddepcontrol.wait
 };
 
 constexpr int SEG_MAX_JOBS = 4;
@@ -177,10 +175,8 @@ __global__ void __launch_bounds__(SegCfg::NT) seg_gemm_kernel(const __grid_const
     const int tid = threadIdx.x;
     const T *Xp = a.X[p], *Vp = a.V[p];
     pdl_trigger();
-    // part 0: every operand word of chunk c; part 1: only the dealer's words (X_0 = U_0 in the
-    // first K segment for party 0, V_p in the second), which were complete before any PDL
-    // predecessor started; part 2: the rest (E, X_1, F: written by the predecessor)
-    auto issue = [&](int c, int part) {
+    pdl_wait();   // operands come from the predecessor
+    auto issue = [&](int c) {
         const int st = c % C::STAGES;
         const int64_t k0 = kbeg + (int64_t)c * C::BK;
 #pragma unroll
@@ -189,8 +185,6 @@ __global__ void __launch_bounds__(SegCfg::NT) seg_gemm_kernel(const __grid_const
             const int64_t m = m0 + mm, k = k0 + kk;
             const bool ok = m < a.M && k < kend;
             const int64_t mc = m < a.M ? m : a.M - 1, kc = k < kend ? k : kend - 1;
-            const bool dealer = kc < K && p == 0;
-            if (part == 1 ? !dealer : part == 2 ? dealer : false) continue;
             const T *src = kc < K ? Xp + mc * K + kc : a.E + mc * K + (kc - K);
             cp_async_elem<sizeof(T)>(As + st * C::A_WORDS + idx, src, ok);
         }
@@ -200,22 +194,13 @@ __global__ void __launch_bounds__(SegCfg::NT) seg_gemm_kernel(const __grid_const
             const int64_t k = k0 + kb, n = n0 + nn;
             const bool ok = n < a.N && k < kend;
             const int64_t kc = k < kend ? k : kend - 1, nc = n < a.N ? n : a.N - 1;
-            const bool dealer = kc >= K;
-            if (part == 1 ? !dealer : part == 2 ? dealer : false) continue;
             const T *src = kc < K ? a.F + kc * a.N + nc : Vp + (kc - K) * a.N + nc;
             cp_async_elem<sizeof(T)>(Bs + st * C::B_WORDS + idx, src, ok);
         }
     };
-    const bool pre = a.dealer_pre != 0;
-    if (pre) {
-#pragma unroll
-        for (int c = 0; c < C::STAGES - 1; ++c)
-            if (c < nch) issue(c, 1);
-    }
-    pdl_wait();   // the (remaining) operands come from the predecessor
 #pragma unroll
     for (int c = 0; c < C::STAGES - 1; ++c) {
-        if (c < nch) issue(c, pre ? 2 : 0);
+        if (c < nch) issue(c);
         cp_async_commit();
     }
     const int tx = tid % C::TX, ty = tid / C::TX;
@@ -227,7 +212,7 @@ __global__ void __launch_bounds__(SegCfg::NT) seg_gemm_kernel(const __grid_const
     for (int c = 0; c < nch; ++c) {
         cp_async_wait<C::STAGES - 2>();
         __syncthreads();
-        if (c + C::STAGES - 1 < nch) issue(c + C::STAGES - 1, 0);
+        if (c + C::STAGES - 1 < nch) issue(c + C::STAGES - 1);
         cp_async_commit();
         const T *as = As + (c % C::STAGES) * C::A_WORDS, *bs = Bs + (c % C::STAGES) * C::B_WORDS;
 #pragma unroll

@@ -741,7 +741,6 @@ static psml_status fused_forward_backward(psml_model_s *m, const T *const X[2], 
         for (int p = 0; p < 2; ++p) { a.V[p] = it.V.p[p]; a.Z[p] = it.Z.p[p]; a.party[p] = p; }
         a.C[0] = C0; a.C[1] = C1;
         a.M = it.M; a.N = it.N; a.K = it.K; a.trunc = trunc; a.nparty = 2;
-        a.dealer_pre = 1;   // U_0, V_p: this step's pool, dealt before the step
         return a;
     };
     // A side of product (l, op): mask U, outputs E, X_1;  B side: mask V, output F
