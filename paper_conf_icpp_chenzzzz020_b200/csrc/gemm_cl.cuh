@@ -29,6 +29,9 @@ struct ClCfg {
     static_assert(SMEM_WORDS >= BM * BN, "reduction buffer must fit");
 };
 using ClDefault = ClCfg<32, 32, 256, 2, 2, 16>;   // measured best on the MLP shapes (tools/micro)
+// the dealer's Z = U V products run beside the online phase: 4 x 4 outputs per thread halve the
+// shared-memory words per ring MAC (PSML_DEAL_TILE=64)
+using ClDealer = ClCfg<64, 64, 256, 4, 4, 16>;
 
 // RingAcc (split-accumulator ring MAC) lives in gemm_simt.cuh, which includes this file.
 

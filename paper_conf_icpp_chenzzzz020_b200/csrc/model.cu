@@ -96,6 +96,7 @@ struct DealPlan {   // fused dealer of one pool (full or inference-only)
     double chacha_blocks = 0;   // ChaCha20 block evaluations of the PRG work list (all streams)
     ClJob<DealerOps<T>> *gemm = nullptr;
     int n_gemm = 0, gemm_ks = 4;
+    bool gemm_big = false;   // 64 x 64 tiles, 4 x 4 per thread (ClDealer) instead of ClDefault
     int64_t gemm_tiles = 0;
     std::vector<int> rest;   // items whose Z = U V runs in its own launch (conv, tcgen05-sized)
 };
@@ -375,7 +376,11 @@ static psml_status build_plan(psml_model_s *m, int pool, bool infer_only) {
         const char *e = getenv("PSML_DEAL_KS");
         const int v = e ? atoi(e) : 4;
         P.gemm_ks = (v == 1 || v == 2 || v == 4 || v == 8) ? v : 4;
+        const char *t = getenv("PSML_DEAL_TILE");   // 64: fewer, more ALU-efficient dealer CTAs
+        P.gemm_big = t && atoi(t) == 64;
     }
+    const int gBM = P.gemm_big ? ClDealer::BM : ClDefault::BM, gBN = P.gemm_big ? ClDealer::BN : ClDefault::BN;
+    const int gBK = P.gemm_big ? ClDealer::BK : ClDefault::BK;
     std::vector<PrgJob> pjm, pjr;   // matrix-triplet streams, then the rest
     std::vector<ClJob<DealerOps<T>>> gj;
     auto job = [&](int kind, std::initializer_list<uint32_t> tags, uint64_t cid, int64_t n,
@@ -409,10 +414,10 @@ static psml_status build_plan(psml_model_s *m, int pool, bool infer_only) {
                 g.ops.U0 = it.U.p[0]; g.ops.U1 = it.U.p[1]; g.ops.V0 = it.V.p[0]; g.ops.V1 = it.V.p[1];
                 g.ops.Z0 = it.Z.p[0]; g.ops.Z1 = it.Z.p[1];
                 g.ops.M = it.M; g.ops.N = it.N; g.ops.Kext = it.K;
-                g.tiles_n = (int)((it.N + ClDefault::BN - 1) / ClDefault::BN);
+                g.tiles_n = (int)((it.N + gBN - 1) / gBN);
                 g.tile_begin = P.gemm_tiles;
-                g.k_per_split = ((it.K + P.gemm_ks - 1) / P.gemm_ks + ClDefault::BK - 1) / ClDefault::BK * ClDefault::BK;
-                P.gemm_tiles += ((it.M + ClDefault::BM - 1) / ClDefault::BM) * g.tiles_n;
+                g.k_per_split = ((it.K + P.gemm_ks - 1) / P.gemm_ks + gBK - 1) / gBK * gBK;
+                P.gemm_tiles += ((it.M + gBM - 1) / gBM) * g.tiles_n;
                 gj.push_back(g);
             } else {
                 P.rest.push_back((int)k);
@@ -522,15 +527,19 @@ static psml_status deal_pool(psml_model_s *m, int pool, uint32_t step, bool infe
         if (P.n_gemm) {
             cudaLaunchConfig_t cfg = {};
             cfg.gridDim = dim3((unsigned)P.gemm_tiles, 1, (unsigned)P.gemm_ks);
-            cfg.blockDim = dim3(ClDefault::NT);
+            cfg.blockDim = dim3(P.gemm_big ? ClDealer::NT : ClDefault::NT);
             cfg.stream = s;
             cudaLaunchAttribute attr[1];
             attr[0].id = cudaLaunchAttributeClusterDimension;
             attr[0].val.clusterDim.x = 1; attr[0].val.clusterDim.y = 1; attr[0].val.clusterDim.z = (unsigned)P.gemm_ks;
             cfg.attrs = attr;
             cfg.numAttrs = 1;
-            PSML_CUDA_TRY(cudaLaunchKernelEx(&cfg, ring_gemm_cl_grouped<T, DealerOps<T>>, (const ClJob<DealerOps<T>> *)P.gemm,
-                                             P.n_gemm, P.gemm_ks));
+            if (P.gemm_big)
+                PSML_CUDA_TRY(cudaLaunchKernelEx(&cfg, ring_gemm_cl_grouped<T, DealerOps<T>, ClDealer>,
+                                                 (const ClJob<DealerOps<T>> *)P.gemm, P.n_gemm, P.gemm_ks));
+            else
+                PSML_CUDA_TRY(cudaLaunchKernelEx(&cfg, ring_gemm_cl_grouped<T, DealerOps<T>>,
+                                                 (const ClJob<DealerOps<T>> *)P.gemm, P.n_gemm, P.gemm_ks));
         }
     }
     for (int k : P.rest) PSML_TRY(deal_gemm(m, m->items[pool][k], s));

@@ -138,6 +138,116 @@ psml_status beaver_matmul_fused(const T *const A[2], const T *const B[2], const 
 // transposed = 1: C = im2col(X)^T . D        M = C*k*k,   K = B*OH*OW, N = Cout
 // ws: 2*nin (raw-input messages) + 2*K*N (F messages) + 2*M*N (split-K)
 // ---------------------------------------------------------------------------------------------
+// Conv weight gradient (the transposed conv product, untruncated: R17 and a9), per image:
+//   C_p[m][n] = Z_p[m][n] + sum_b sum_(oy,ox) (p E + U_p)[b, src(m) + oy W + ox] F[(b,oy,ox)][n]
+//                                           +  E[b, src(m) + oy W + ox]        V_p[(b,oy,ox)][n]
+// with E = mE0 + mE1 and F = mF0 + mF1 (the opened messages) and src(m) = coloff[m], m = (ch, ky,
+// kx) -- the same sum as ConvBeaverOps with transposed = 1, regrouped by image.  One CTA = one
+// (image, party, half of the output rows): the image's operand plane and the half's F (or V) rows
+// sit in shared memory, thread (m, n-quad) runs its 4 split accumulators over the half's output
+// positions, and the partial tile is added to C_p (pre-set to Z_p) with 64-bit atomics (ring
+// addition is exact, so the order does not matter: bit-identical to the generic GEMM, tested).
+template <typename T>
+__global__ void __launch_bounds__(1024) conv_gw_image_kernel(const T *__restrict__ mE0, const T *__restrict__ mE1,
+                                                             const T *__restrict__ U0, const T *__restrict__ U1,
+                                                             const T *__restrict__ mF0, const T *__restrict__ mF1,
+                                                             const T *__restrict__ V0, const T *__restrict__ V1,
+                                                             ConvGeom g, int64_t N, T *C0, T *C1) {
+    extern __shared__ __align__(16) unsigned char conv_smem[];
+    T *img = (T *)conv_smem;
+    const int chw = g.C * g.H * g.W;
+    const int b = blockIdx.x, p = blockIdx.y, half = blockIdx.z;
+    const int oy0 = half * ((g.OH + 1) / 2), oy1 = min(g.OH, oy0 + (g.OH + 1) / 2);
+    const int npos = (oy1 - oy0) * g.OW;
+    T *fb = img + chw;
+    const int M = g.C * g.k * g.k, NQ = (int)N / 4;
+    const int t = threadIdx.x;
+    const bool act = t < M * NQ;
+    const int m = act ? t % M : 0, nq = act ? t / M : 0;
+    const int off = act ? g.coloff[m] : 0;
+    RingAcc<T> acc[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) acc[j].zero();
+    const T *ub = (p ? U1 : U0) + (int64_t)b * chw;
+    const T *vb = (p ? V1 : V0);
+    const int64_t r0 = (int64_t)b * g.OH * g.OW + (int64_t)oy0 * g.OW;   // first im2col row of the half
+    for (int seg = 0; seg < 2; ++seg) {
+        // operand plane: segment 0 -> p E + U_p, segment 1 -> E; rows: segment 0 -> F, 1 -> V_p
+        for (int i = t; i < chw; i += blockDim.x) {
+            const int64_t gi = (int64_t)b * chw + i;
+            const T e = mE0[gi] + mE1[gi];
+            img[i] = seg == 0 ? (T)((T)p * e + ub[i]) : e;
+        }
+        for (int i = t; i < npos * (int)N; i += blockDim.x) {
+            const int64_t gi = r0 * N + i;
+            fb[i] = seg == 0 ? (T)(mF0[gi] + mF1[gi]) : vb[gi];
+        }
+        __syncthreads();
+        if (act) {
+            for (int oy = oy0; oy < oy1; ++oy) {
+                const T *arow = img + off + oy * g.W;
+                const T *brow = fb + (int64_t)(oy - oy0) * g.OW * N + 4 * nq;
+#pragma unroll 4
+                for (int ox = 0; ox < g.OW; ++ox) {
+                    const T a = arow[ox];
+                    const ulonglong2 b01 = *(const ulonglong2 *)(brow + ox * N);
+                    const ulonglong2 b23 = *(const ulonglong2 *)(brow + ox * N + 2);
+                    acc[0].mac(a, (T)b01.x); acc[1].mac(a, (T)b01.y);
+                    acc[2].mac(a, (T)b23.x); acc[3].mac(a, (T)b23.y);
+                }
+            }
+        }
+        __syncthreads();
+    }
+    if (act) {
+        T *c = (p ? C1 : C0) + (int64_t)m * N + 4 * nq;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) atomicAdd((unsigned long long *)(c + j), (unsigned long long)acc[j].value());
+    }
+}
+
+// PSML_CONV_GW=generic keeps the weight gradient on the generic im2col GEMM (tests)
+inline bool conv_gw_enabled() {
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("PSML_CONV_GW");
+        v = (e && e[0] == 'g') ? 0 : 1;
+    }
+    return v == 1;
+}
+
+// The fast path applies to the untruncated weight gradient in Z_2^64 with N % 4 == 0 and
+// operands that fit shared memory; false -> the generic im2col GEMM.
+template <typename T>
+bool conv_gw_fast_ok(const ConvGeom &g, int64_t N, int transposed, int trunc) {
+    if (sizeof(T) != 8 || !transposed || trunc != 0 || N % 4 != 0) return false;
+    const int64_t M = (int64_t)g.C * g.k * g.k;
+    if (M * (N / 4) > 1024) return false;
+    const int64_t words = (int64_t)g.C * g.H * g.W + (int64_t)((g.OH + 1) / 2) * g.OW * N;
+    return words * (int64_t)sizeof(T) <= 200 * 1024;
+}
+
+template <typename T>
+psml_status conv_gw_fast(const T *mE0, const T *mE1, const T *const UX[2], const T *mF0, const T *mF1,
+                         const T *const V[2], const T *const Z[2], int64_t batch, const ConvGeom &g, int64_t N,
+                         T *const C[2], cudaStream_t s) {
+    const int64_t M = (int64_t)g.C * g.k * g.k;
+    for (int p = 0; p < 2; ++p)
+        PSML_CUDA_TRY(cudaMemcpyAsync(C[p], Z[p], sizeof(T) * (size_t)(M * N), cudaMemcpyDeviceToDevice, s));
+    const size_t smem = sizeof(T) * (size_t)((int64_t)g.C * g.H * g.W + (int64_t)((g.OH + 1) / 2) * g.OW * N);
+    static bool attr = false;
+    if (!attr) {
+        PSML_CUDA_TRY(cudaFuncSetAttribute(conv_gw_image_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                           200 * 1024));
+        attr = true;
+    }
+    const int threads = (int)((M * (N / 4) + 31) / 32 * 32);
+    conv_gw_image_kernel<T><<<dim3((unsigned)batch, 2, 2), threads, smem, s>>>(mE0, mE1, UX[0], UX[1], mF0, mF1,
+                                                                               V[0], V[1], g, N, C[0], C[1]);
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
 template <typename T>
 psml_status conv_beaver(const T *const X[2], const T *const Bm[2], const T *const UX[2],
                         const T *const V[2], const T *const Z[2], int64_t batch, ConvGeom g,
@@ -156,6 +266,8 @@ psml_status conv_beaver(const T *const X[2], const T *const Bm[2], const T *cons
     const int64_t maxt = std::max(((batch + 31) / 32) * (((int64_t)g.C * g.H * g.W + 31) / 32), ((K + 31) / 32) * ((N + 31) / 32));
     mask_kernel<T><<<dim3((unsigned)std::min<int64_t>(maxt, 148 * 8), 1, 4), dim3(32, 8), 0, s>>>(jobs);
     PSML_LAUNCH_CHECK();
+    if (conv_gw_fast_ok<T>(g, N, transposed, trunc) && conv_gw_enabled())
+        return conv_gw_fast<T>(mE0, mE1, UX, mF0, mF1, V, Z, batch, g, N, C, s);
     ConvBeaverOps<T> ops;
     ops.mE0 = mE0; ops.mE1 = mE1; ops.mF0 = mF0; ops.mF1 = mF1;
     for (int p = 0; p < 2; ++p) { ops.UX[p] = UX[p]; ops.V[p] = V[p]; ops.Z[p] = Z[p]; ops.C[p] = C[p]; }

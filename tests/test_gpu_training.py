@@ -170,15 +170,17 @@ def test_explicit_mask_round_matches_fused_open():
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
 
 
-@pytest.mark.parametrize("env", [{"PSML_SEG": "simt"}, {"PSML_SEG": "tc"}, {"PSML_ROWS": "0"},
+@pytest.mark.parametrize("env", [{"PSML_SEG": "simt"}, {"PSML_SEG": "tc"}, {"PSML_ROWS": "0", "PSML_CONV_GW": "generic"},
                                  {"PSML_DEAL_AFTER": "0", "PSML_DEAL_SPLIT": "0"},
-                                 {"PSML_DEAL_AFTER": "4", "PSML_DEAL_CTAS": "0"}],
-                         ids=["seg_simt", "seg_tc", "rows_off", "deal_at_fork_one_branch", "deal_late_full_grid"])
+                                 {"PSML_DEAL_AFTER": "4", "PSML_DEAL_CTAS": "0", "PSML_DEAL_TILE": "64"}],
+                         ids=["seg_simt", "seg_tc", "rows_off_conv_gw_generic", "deal_at_fork_one_branch", "deal_late_full_grid_tile64"])
 def test_seg_gemm_backends_match_oracle(env):
     """PSML_SEG=simt: every opened Beaver product of the training step on the CUDA-core
     two-segment GEMM; PSML_SEG=tc: every eligible one on the tcgen05 in-kernel-split GEMM
     (gemm_tcseg.cu; by default only groups of >= 2^25 ring MACs go there); PSML_ROWS=0: the CNN's
-    tall-skinny conv products on the 16 x 16 small-tile kernel instead of ring_gemm_rows;
+    tall-skinny conv products on the 16 x 16 small-tile kernel instead of ring_gemm_rows, and
+    PSML_CONV_GW=generic the conv weight gradient on the generic im2col GEMM instead of the
+    per-image kernel;
     PSML_DEAL_AFTER / PSML_DEAL_SPLIT / PSML_DEAL_CTAS: where the pipelined graph forks the next
     step's dealer from the online chain, whether its PRG runs as one or two branches, and its grid.
     All reproduce the oracle exactly."""
