@@ -138,24 +138,31 @@ __device__ __forceinline__ void cl_finish(const Ops &ops, int p, int64_t m0, int
     }
     namespace cg = cooperative_groups;
     cg::cluster_group cluster = cg::this_cluster();
+    const int rank = (int)cluster.block_rank();
+    constexpr int MAXC = (BM * BN + 2 * NT - 1) / (2 * NT);   // ks >= 2
+    const int per = (BM * BN) / ks;                              // ks divides BM * BN (power of two)
+    T sum[MAXC], zz[MAXC];
+    // this CTA's epilogue Z words first: their load latency overlaps the partial-tile exchange
+#pragma unroll
+    for (int u = 0; u < MAXC; ++u) {
+        zz[u] = 0;
+        if (tid + u * NT < per) {
+            const int e = rank * per + tid + u * NT;
+            const int64_t m = m0 + e / BN, n = n0 + e % BN;
+            zz[u] = ops.zload(p, m < ops.M ? m : ops.M - 1, n < ops.N ? n : ops.N - 1);
+        }
+    }
     __syncthreads();   // all warps done with the operand tiles that `red` overlays
 #pragma unroll
     for (int i = 0; i < C::TM; ++i)
 #pragma unroll
         for (int j = 0; j < C::TN; ++j) red[(ty + i * (BM / C::TM)) * BN + tx + j * C::TX] = acc[i][j];
     cluster.sync();
-    const int rank = (int)cluster.block_rank();
-    constexpr int MAXC = (BM * BN + 2 * NT - 1) / (2 * NT);   // ks >= 2
-    const int per = (BM * BN) / ks;                              // ks divides BM * BN (power of two)
-    T sum[MAXC], zz[MAXC];
 #pragma unroll
     for (int u = 0; u < MAXC; ++u) {
         sum[u] = 0;
-        zz[u] = 0;
         if (tid + u * NT < per) {
             const int e = rank * per + tid + u * NT;
-            const int64_t m = m0 + e / BN, n = n0 + e % BN;
-            zz[u] = ops.zload(p, m < ops.M ? m : ops.M - 1, n < ops.N ? n : ops.N - 1);
             T part[8];
 #pragma unroll
             for (int q = 0; q < 8; ++q) part[q] = q < ks ? cluster.map_shared_rank(red, q)[e] : (T)0;
@@ -171,7 +178,9 @@ __device__ __forceinline__ void cl_finish(const Ops &ops, int p, int64_t m0, int
             if (m < ops.M && n < ops.N) ops.put(p, m, n, sum[u], zz[u]);
         }
     }
-    cluster.sync();    // peers' shared memory stays alive until every CTA has read it
+    // peers' shared memory stays alive until every CTA has read it (the reads completed: their
+    // values were summed above), so no memory ordering is needed here
+    asm volatile("barrier.cluster.arrive.relaxed.aligned;\nbarrier.cluster.wait.aligned;" ::: "memory");
 }
 
 // One product: grid (ceil(N/BN), ceil(M/BM), nparty * ks), cluster (1, 1, ks).
