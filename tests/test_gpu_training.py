@@ -125,6 +125,47 @@ def test_step_host_bitexact_vs_oracle(T, task):
     tr.close()
 
 
+@pytest.mark.parametrize("task", ["mlp", "logreg"])
+def test_one_epoch_bench_path_bitexact_vs_eager_and_fp64(T, task):
+    """The launch configuration bench.py times -- pipelined CUDA graph (dealer of step s+1 forked
+    from the online chain of step s), fed through psml_model_step_host from pinned 8-bit pixels --
+    over a whole epoch (468 steps of 128): master-weight shares bit-identical to the eager
+    per-kernel path (whose steps the oracle pins exactly, test_training_bitexact_vs_oracle), and
+    decoded weights within 2^-12 of fp64 SGD."""
+    Wi = synth.init_weights(task)
+    steps = 60000 // 128
+    eager = T.SecureTrainer(task, Wi, backend=0)
+    for s in range(steps):
+        X, Y = synth.batch(task, s)
+        eager.step(torch.from_numpy(X), torch.from_numpy(Y), s)
+    want = [tuple(to_np(w).copy() for w in eager.master_shares(l)) for l in range(len(Wi))]
+    eager.close()
+    tr = T.SecureTrainer(task, Wi, backend=0)
+    pm = plain.PlainModel(task, Wi)
+    X, Y = synth.batch(task, 0)
+    tr.step(torch.from_numpy(X), torch.from_numpy(Y), 0)
+    pm.step(X, Y)
+    tr.capture(pipelined=True)
+    out = None
+    for s in range(1, steps):
+        q, y = synth.batch_u8(task, s)
+        qh, yh = torch.from_numpy(q).pin_memory(), torch.from_numpy(np.ascontiguousarray(y)).pin_memory()
+        if out is None:
+            out = torch.empty((2, q.shape[0], tr.out_dim), dtype=torch.uint64).pin_memory()
+        tr.graph_step_host(qh, yh, s, out)
+        torch.cuda.synchronize()   # the pinned inputs are reused by the next iteration
+        X, Y = synth.batch(task, s)
+        pm.step(X, Y)
+    for l in range(len(Wi)):
+        g0, g1 = tr.master_shares(l)
+        assert np.array_equal(to_np(g0), want[l][0]) and np.array_equal(to_np(g1), want[l][1]), l
+    got = [w.cpu().numpy() for w in tr.master_weights()]
+    err = max(np.abs(g.reshape(w.shape) - w).max() for g, w in zip(got, pm.W))
+    print(f"{task} (bench path): one-epoch max |w - w_fp64| = 2^{np.log2(err):.2f}")
+    assert err < 2.0 ** -12
+    tr.close()
+
+
 def test_cnn_one_epoch_against_fp64(T):
     """Config 4 (CIFAR-shaped CNN, 390 steps of 128): decoded master weights vs fp64 SGD.
 
