@@ -80,10 +80,16 @@ class ClockSampler:
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", "-i", str(self.index), "--query-gpu=clocks.sm,clocks.max.sm,"
-                 "clocks_event_reasons.active", "--format=csv,noheader,nounits", "-lms", "25"],
+                 "clocks_event_reasons.active", "--format=csv,noheader,nounits", "-lms", "20"],
                 stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.thread = threading.Thread(target=self._read, daemon=True)
             self.thread.start()
+            # nvidia-smi takes a while to start: wait for its first sample so the sampling is live
+            # when the timed region begins, then keep only samples taken inside the region
+            t0 = time.time()
+            while not self.samples and time.time() - t0 < 15.0 and self.proc.poll() is None:
+                time.sleep(0.01)
+            self.samples.clear()
         except OSError:
             self.proc = None
         return self
