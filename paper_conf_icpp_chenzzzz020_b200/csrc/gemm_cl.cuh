@@ -113,9 +113,44 @@ __device__ __forceinline__ void cl_tile(const Ops &ops, int p, int64_t m0, int64
 }
 
 // Store (KS == 1) or cluster-reduce + store one tile.  `red` = this CTA's smem (>= BM x BN words).
+// Epilogue Z words of this thread (the order cl_finish consumes them), for kernels that load them
+// ahead of time (before griddepcontrol.wait): ks == 1 -> TM x TN outputs of the thread; ks > 1 ->
+// the thread's elements of this CTA's 1/ks slice of the reduced tile.
+template <class C> constexpr int cl_zpre_n() {
+    return C::TM * C::TN > (C::BM * C::BN + 2 * C::NT - 1) / (2 * C::NT) ? C::TM * C::TN
+                                                                       : (C::BM * C::BN + 2 * C::NT - 1) / (2 * C::NT);
+}
+template <typename T, class Ops, class C>
+__device__ __forceinline__ void cl_zload(const Ops &ops, int p, int64_t m0, int64_t n0, int ks, int rank,
+                                         T z[cl_zpre_n<C>()]) {
+    constexpr int BM = C::BM, BN = C::BN, NT = C::NT;
+    const int tid = threadIdx.x, tx = tid % C::TX, ty = tid / C::TX;
+    if (ks == 1) {
+#pragma unroll
+        for (int i = 0; i < C::TM; ++i)
+#pragma unroll
+            for (int j = 0; j < C::TN; ++j) {
+                const int64_t m = m0 + ty + i * (BM / C::TM), n = n0 + tx + j * C::TX;
+                z[i * C::TN + j] = ops.zload(p, m < ops.M ? m : ops.M - 1, n < ops.N ? n : ops.N - 1);
+            }
+        return;
+    }
+    constexpr int MAXC = (BM * BN + 2 * NT - 1) / (2 * NT);
+    const int per = (BM * BN) / ks;
+#pragma unroll
+    for (int u = 0; u < MAXC; ++u) {
+        z[u] = 0;
+        if (tid + u * NT < per) {
+            const int e = rank * per + tid + u * NT;
+            const int64_t m = m0 + e / BN, n = n0 + e % BN;
+            z[u] = ops.zload(p, m < ops.M ? m : ops.M - 1, n < ops.N ? n : ops.N - 1);
+        }
+    }
+}
+
 template <typename T, class Ops, class C>
 __device__ __forceinline__ void cl_finish(const Ops &ops, int p, int64_t m0, int64_t n0, int ks, T *red,
-                                          T acc[C::TM][C::TN]) {
+                                          T acc[C::TM][C::TN], const T *zpre = nullptr) {
     constexpr int BM = C::BM, BN = C::BN, NT = C::NT;
     const int tid = threadIdx.x, tx = tid % C::TX, ty = tid / C::TX;
     if (ks == 1) {   // epilogue operands first (clamped, unconditional), then the stores
@@ -125,7 +160,7 @@ __device__ __forceinline__ void cl_finish(const Ops &ops, int p, int64_t m0, int
 #pragma unroll
             for (int j = 0; j < C::TN; ++j) {
                 const int64_t m = m0 + ty + i * (BM / C::TM), n = n0 + tx + j * C::TX;
-                z[i][j] = ops.zload(p, m < ops.M ? m : ops.M - 1, n < ops.N ? n : ops.N - 1);
+                z[i][j] = zpre ? zpre[i * C::TN + j] : ops.zload(p, m < ops.M ? m : ops.M - 1, n < ops.N ? n : ops.N - 1);
             }
 #pragma unroll
         for (int i = 0; i < C::TM; ++i)
@@ -149,7 +184,7 @@ __device__ __forceinline__ void cl_finish(const Ops &ops, int p, int64_t m0, int
         if (tid + u * NT < per) {
             const int e = rank * per + tid + u * NT;
             const int64_t m = m0 + e / BN, n = n0 + e % BN;
-            zz[u] = ops.zload(p, m < ops.M ? m : ops.M - 1, n < ops.N ? n : ops.N - 1);
+            zz[u] = zpre ? zpre[u] : ops.zload(p, m < ops.M ? m : ops.M - 1, n < ops.N ? n : ops.N - 1);
         }
     }
     __syncthreads();   // all warps done with the operand tiles that `red` overlays

@@ -175,6 +175,12 @@ __global__ void __launch_bounds__(SegCfg::NT) seg_gemm_kernel(const __grid_const
     const int tid = threadIdx.x;
     const T *Xp = a.X[p], *Vp = a.V[p];
     pdl_trigger();
+    // the epilogue's Z_p words are dealer material, complete before any PDL predecessor started
+    // (dealer kernels never trigger early): load them while the predecessor finishes
+    SegEpi<T> epi{&a, a.M, a.N};
+    T zpre[cl_zpre_n<C>()];
+    cl_zload<T, SegEpi<T>, C>(epi, p, m0, n0, ks, ks > 1 ? (int)cooperative_groups::this_cluster().block_rank() : 0,
+                              zpre);
     pdl_wait();   // operands come from the predecessor
     auto issue = [&](int c) {
         const int st = c % C::STAGES;
@@ -234,8 +240,7 @@ __global__ void __launch_bounds__(SegCfg::NT) seg_gemm_kernel(const __grid_const
     for (int i = 0; i < C::TM; ++i)
 #pragma unroll
         for (int j = 0; j < C::TN; ++j) acc[i][j] = r[i][j].value();
-    SegEpi<T> epi{&a, a.M, a.N};
-    cl_finish<T, SegEpi<T>, C>(epi, p, m0, n0, ks, smem, acc);
+    cl_finish<T, SegEpi<T>, C>(epi, p, m0, n0, ks, smem, acc, zpre);
 }
 
 // tcgen05 form of the same group (gemm_tcseg.cu; l = 64, sm_100, K' <= 16384 per product).
