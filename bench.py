@@ -687,8 +687,21 @@ def cpu_baseline(budget_s=12.0):
     t1, cores = oracle_steps(1, base=10000)
     n = max(2, min(60, int(budget_s / max(t1, 1e-3))))
     t, cores = oracle_steps(n, base=10001)
-    return {"value": BATCH * n / t, "unit": "samples/s", "cores": cores, "kind": "oracle",
-            "sample": f"{n} full oracle secure MLP training steps (batch 128) on the host"}
+    out = {"value": BATCH * n / t, "unit": "samples/s", "cores": cores, "kind": "oracle",
+           "sample": f"{n} full oracle secure MLP training steps (batch 128) on the host"}
+    # the same oracle on ONE host thread (nproc and 1 thread), a few steps in a
+    # subprocess with OMP_NUM_THREADS=1
+    try:
+        code = ("import sys, json; sys.path.insert(0, %r); import bench; "
+                "t, c = bench.oracle_steps(%d, base=10100); print(json.dumps([t, c]))" % (ROOT, 3))
+        r = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=300,
+                           env=dict(os.environ, OMP_NUM_THREADS="1"), cwd=ROOT)
+        t1s, c1 = json.loads(r.stdout.strip().splitlines()[-1])
+        out["one_thread"] = {"value": BATCH * 3 / t1s, "unit": "samples/s", "cores": c1,
+                             "sample": "3 full oracle secure MLP training steps, OMP_NUM_THREADS=1"}
+    except Exception as e:  # noqa: BLE001 -- reported, never fatal
+        out["one_thread"] = {"unavailable": str(e)[:200]}
+    return out
 
 
 # ---------------------------------------------------------------------------------------------
