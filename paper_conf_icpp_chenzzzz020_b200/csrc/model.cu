@@ -479,15 +479,19 @@ static cudaStream_t deal_s2(psml_model_s *m) {
 
 // PRG jobs [j0, j1) (blocks [b0, b1)) of plan P on stream s
 static psml_status deal_prg_launch(psml_model_s *m, const DealPlan &P, int j0, int j1, int64_t b0, int64_t b1,
-                                   cudaStream_t s) {
+                                   cudaStream_t s, bool second = false) {
     if (j1 <= j0 || b1 <= b0) return PSML_OK;
     // a bounded grid (grid-stride): the PRG work runs beside the online phase instead of
-    // occupying every SM's register file ahead of it (PSML_DEAL_CTAS per SM; 0 = full grid)
-    static int per_sm = -1;
-    if (per_sm < 0) {
+    // occupying every SM's register file ahead of it (PSML_DEAL_CTAS per SM; 0 = full grid;
+    // PSML_DEAL_CTAS2 for the second dealer branch)
+    static int per_sm1 = -1, per_sm2 = -1;
+    if (per_sm1 < 0) {
         const char *e = getenv("PSML_DEAL_CTAS");
-        per_sm = e ? atoi(e) : 4;   // measured best of {1, 2, 4, full} (tools/gpu44.sh)
+        per_sm1 = e ? atoi(e) : 4;   // measured best of {1, 2, 4, full} (tools/gpu44.sh)
+        const char *e2 = getenv("PSML_DEAL_CTAS2");
+        per_sm2 = e2 ? atoi(e2) : std::min(per_sm1, 2);   // tools/gpu92.sh: 2 best of {2, 3, 4}
     }
+    const int per_sm = second ? per_sm2 : per_sm1;
     const int64_t full = (b1 - b0 + 127) / 128;
     // a dealer forked after the whole online chain (models without the fused step, e.g. the CNN)
     // overlaps nothing but the update: it takes the whole GPU
@@ -516,11 +520,13 @@ static psml_status deal_pool(psml_model_s *m, int pool, uint32_t step, bool infe
     {
         ProfScope prof(PROF_DEALER, s, P.chacha_blocks);   // work = ChaCha20 blocks of the step
         if (fork) {
+            // the matrix-triplet streams (needed by the Z = U V launch that follows them) are
+            // created first so they are scheduled first; the second branch forks from before them
             PSML_CUDA_TRY(cudaEventRecord(m->ev_d2, s));
-            PSML_CUDA_TRY(cudaStreamWaitEvent(s2, m->ev_d2, 0));
-            PSML_TRY(deal_prg_launch(m, P, P.n_prg_mat, P.n_prg, P.prg_mat_blocks, P.prg_blocks, s2));
-            PSML_CUDA_TRY(cudaEventRecord(m->ev_d2j, s2));
             PSML_TRY(deal_prg_launch(m, P, 0, P.n_prg_mat, 0, P.prg_mat_blocks, s));
+            PSML_CUDA_TRY(cudaStreamWaitEvent(s2, m->ev_d2, 0));
+            PSML_TRY(deal_prg_launch(m, P, P.n_prg_mat, P.n_prg, P.prg_mat_blocks, P.prg_blocks, s2, true));
+            PSML_CUDA_TRY(cudaEventRecord(m->ev_d2j, s2));
         } else {
             PSML_TRY(deal_prg_launch(m, P, 0, P.n_prg, 0, P.prg_blocks, s));
         }
