@@ -1,0 +1,12 @@
+cd $GRAFT_REPO_ROOT
+mkdir -p gpurun_out
+( timeout 2400 python -m pytest tests -m gpu -x -q ) > gpurun_out/t94.log 2>&1; tail -2 gpurun_out/t94.log
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" 2>&1 | tail -1
+timeout 900 python bench.py > gpurun_out/b94.json 2> gpurun_out/b94.err
+python -c "
+import json; d=json.load(open('gpurun_out/b94.json'))
+print('value',round(d['value']),'e2e',round(d['e2e']['value']),'online_graph',round(d['online_graph_samples_per_s']),'ms',round(d['ms_per_step'],4), d['clocks'], d['roofline']['frac'], d['cpu_baseline'])"
+timeout 900 python bench.py --task cnn --steps 200 --no-cpu-baseline --no-ring-gemm > gpurun_out/b94c.json 2> gpurun_out/b94c.err
+python -c "
+import json; d=json.load(open('gpurun_out/b94c.json'))
+print('cnn value',round(d['value']),'e2e',round(d['e2e']['value']),'online',round(d['online_samples_per_s']),'ms',round(d['ms_per_step'],4))"
