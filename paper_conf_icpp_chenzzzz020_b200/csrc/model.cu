@@ -1508,6 +1508,41 @@ psml_status psml_model_capture_step(psml_model m, const void *const X[2], const 
     return PSML_OK;
 }
 
+// Client encode + share of a whole minibatch in one launch (psml_model_step_host, Z_2^64): ChaCha20
+// blocks [0, nx/8) share X from 8-bit pixels (x = q / 255), the rest share Y from class indices
+// (one-hot) or float64 labels -- the same words as psml_encode_share_u8 / _onehot / encode_share.
+struct ClientJob {
+    PrgKey kx, ky;
+    const uint8_t *q;
+    const uint8_t *ycls;
+    const double *yf;
+    int64_t nx, ny, classes;
+    int f;
+    uint64_t *x0, *x1, *y0, *y1;
+};
+__global__ void __launch_bounds__(128) client_share_kernel(const ClientJob j) {
+    const int64_t bx = (j.nx + 7) / 8, total = bx + (j.ny + 7) / 8;
+    for (int64_t g = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; g < total; g += (int64_t)gridDim.x * blockDim.x) {
+        const bool isx = g < bx;
+        const int64_t b = isx ? g : g - bx, n = isx ? j.nx : j.ny;
+        uint32_t w[16];
+        chacha20_block(isx ? j.kx : j.ky, (uint32_t)b, w);
+#pragma unroll
+        for (int t = 0; t < 8; ++t) {
+            const int64_t e = b * 8 + t;
+            if (e >= n) break;
+            double x;
+            if (isx) x = (double)j.q[e] / 255.0;
+            else if (j.ycls) x = (int64_t)j.ycls[e / j.classes] == e % j.classes ? 1.0 : 0.0;
+            else x = j.yf[e];
+            const uint64_t r = ((uint64_t)w[2 * t + 1] << 32) | w[2 * t];
+            const uint64_t v = (uint64_t)(unsigned long long)__double2ll_rn(ldexp(x, j.f));
+            (isx ? j.x0 : j.y0)[e] = r;
+            (isx ? j.x1 : j.y1)[e] = v - r;
+        }
+    }
+}
+
 // out[0..n) = a, out[n..2n) = b (the prediction shares into mapped host memory)
 template <typename U>
 __global__ void copy_pair_kernel(const U *__restrict__ a, const U *__restrict__ b, int64_t n, U *__restrict__ out) {
@@ -1552,13 +1587,29 @@ psml_status psml_model_step_host(psml_model m, const uint8_t *q, const void *y, 
     }
     const psml_ring ring = m->ctx->ring;
     const uint64_t cx = call_id(m->d.pair_id, step_id, 0, OP_SHARE, 0), cy = call_id(m->d.pair_id, step_id, 0, OP_SHARE, 1);
-    PSML_TRY(psml_encode_share_u8(ring, share_seed, cx, qd, nx, 255.0, (void *)m->cap_X[0], (void *)m->cap_X[1], stream));
-    if (y_kind)
-        PSML_TRY(psml_encode_share_onehot(ring, share_seed, cy, (const uint8_t *)yd, m->B, dl, (void *)m->cap_Y[0],
-                                          (void *)m->cap_Y[1], stream));
-    else
-        PSML_TRY(psml_encode_share(ring, share_seed, cy, (const double *)yd, ny, (void *)m->cap_Y[0],
-                                   (void *)m->cap_Y[1], stream));
+    if (ring.l == 64 && nx > 0 && ny > 0) {
+        // X and Y in one launch: one PCIe round trip for the mapped host reads instead of two
+        ClientJob cj{};
+        cj.kx = make_key(share_seed, TAG_SH, cx);
+        cj.ky = make_key(share_seed, TAG_SH, cy);
+        cj.q = qd; cj.nx = nx; cj.f = ring.frac_bits;
+        cj.ycls = y_kind ? (const uint8_t *)yd : nullptr;
+        cj.yf = y_kind ? nullptr : (const double *)yd;
+        cj.ny = ny; cj.classes = dl;
+        cj.x0 = (T *)m->cap_X[0]; cj.x1 = (T *)m->cap_X[1]; cj.y0 = (T *)m->cap_Y[0]; cj.y1 = (T *)m->cap_Y[1];
+        const int64_t blocks = (nx + 7) / 8 + (ny + 7) / 8;
+        client_share_kernel<<<grid_for(blocks, 128), 128, 0, s>>>(cj);
+        PSML_LAUNCH_CHECK();
+    } else {
+        PSML_TRY(psml_encode_share_u8(ring, share_seed, cx, qd, nx, 255.0, (void *)m->cap_X[0], (void *)m->cap_X[1],
+                                      stream));
+        if (y_kind)
+            PSML_TRY(psml_encode_share_onehot(ring, share_seed, cy, (const uint8_t *)yd, m->B, dl, (void *)m->cap_Y[0],
+                                              (void *)m->cap_Y[1], stream));
+        else
+            PSML_TRY(psml_encode_share(ring, share_seed, cy, (const double *)yd, ny, (void *)m->cap_Y[0],
+                                       (void *)m->cap_Y[1], stream));
+    }
     // servers: the captured step
     PSML_TRY(psml_model_step_graph(m, step_id, stream));
     // client: both parties' prediction shares back
