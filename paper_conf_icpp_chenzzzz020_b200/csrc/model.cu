@@ -1241,7 +1241,11 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
         // work fills the SMs they leave idle (PSML_PRIO=0 disables)
         int lo = 0, hi = 0;
         PSML_CUDA_TRY(cudaDeviceGetStreamPriorityRange(&lo, &hi));
-        PSML_CUDA_TRY(cudaStreamCreateWithPriority(&m->side, cudaStreamNonBlocking, lo));
+        // PSML_DEAL_PRIO1: priority of the first dealer branch (matrix-triplet PRG + Z = U V, which
+        // the step's end waits for) as steps above the lowest; default the lowest
+        int p1 = lo;
+        if (const char *e = getenv("PSML_DEAL_PRIO1")) p1 = std::max(hi, lo - std::max(0, atoi(e)));
+        PSML_CUDA_TRY(cudaStreamCreateWithPriority(&m->side, cudaStreamNonBlocking, p1));
         PSML_CUDA_TRY(cudaStreamCreateWithPriority(&m->side2, cudaStreamNonBlocking, lo));
         PSML_CUDA_TRY(cudaStreamCreateWithPriority(&m->hi, cudaStreamNonBlocking, hi));
         PSML_CUDA_TRY(cudaStreamCreateWithPriority(&m->gw, cudaStreamNonBlocking, hi));
