@@ -251,7 +251,7 @@ def bench_ours(args):
         gs.wait_stream(stream)
         with torch.cuda.stream(gs):
             tr.model.capture_step(tr.Xbuf, tr.Ybuf, with_deal=False, with_update=True, pipelined=False,
-                                  stream=gs)
+                                  stream=gs, unsafe_reuse_material=True)
         stream.wait_stream(gs)
         tr.model.step_graph(0)
         torch.cuda.synchronize()

@@ -299,6 +299,11 @@ psml_status psml_train_apply_update(psml_model model, int32_t extra_shift, psml_
  * dealer of step s + 1 on a forked stream concurrently with the online phase of step s (the first
  * step's pool must be filled with psml_model_deal).  The dealer's call ids take their step field
  * from a model-owned device word, so the same graph(s) serve every step.
+ * Without bit 0 the graph consumes material dealt by psml_model_deal for exactly the replayed
+ * step id (one graph per pool), once: dealer material is single-use (a mask opened on two values
+ * leaks their difference), and the eager calls consume it the same way.  Bit 3 (only without
+ * bits 0 and 2) = UNSAFE benchmark-only replay of pool 0 as last dealt, for timing the online
+ * phase alone; never used for training.
  * psml_model_step_graph writes the step word and launches the graph; the caller refills X/Y
  * before each replay; pipelined steps must be consecutive (PSML_ERR_STATE otherwise).
  * Capture must not overlap other work on the stream. */
@@ -349,12 +354,43 @@ psml_status psml_nccl_unique_id(uint8_t uid[128]);
  * step's stream (stream-ordered, no host synchronisation; NVLink P2P between GPUs). */
 psml_status psml_xport_nccl_create(const uint8_t uid[128], int32_t rank, psml_xport *out);
 psml_status psml_xport_callback_create(psml_exchange_fn fn, void *user, psml_xport *out);
+/* Peer-memory transport (the B200-native one).  Each party allocates a
+ * double-buffered mailbox of 2 x capacity_bytes (+ a few flag words) in its own HBM and exports
+ * a PSML_PEER_HANDLE_BYTES blob (CUDA IPC handles + process id); the caller ships the blob to the
+ * peer (e.g. all_gather over a torch.distributed group) and both call psml_xport_peer_connect
+ * with the other party's blob.  The peer's mailbox is then mapped into this process (CUDA IPC:
+ * NVLink P2P between two GPUs, the same HBM for two processes on one GPU; a raw pointer when
+ * both parties live in one process).  One exchange is ONE kernel on the caller's stream: it
+ * stores this party's messages into the peer's mailbox, releases a sequence number into the
+ * peer's flag word (system scope), waits for the peer's, and copies its own mailbox out to
+ * `recv` -- no host synchronisation, and graph-capturable (sequence numbers live in device
+ * memory).  An exchange larger than capacity_bytes runs as several mailbox rounds.  Both
+ * parties must issue the same exchanges in the same order (like NCCL collectives); a peer that
+ * stops answering makes the kernel trap after 60 s (PSML_ERR_CUDA on the next call) instead of
+ * hanging the GPU.  party: 0 or 1; capacity_bytes >= 4096, equal on both sides. */
+#define PSML_PEER_HANDLE_BYTES 256
+psml_status psml_xport_peer_create(int32_t party, int64_t capacity_bytes, psml_xport *out,
+                                   uint8_t handle[PSML_PEER_HANDLE_BYTES]);
+psml_status psml_xport_peer_connect(psml_xport x, const uint8_t peer_handle[PSML_PEER_HANDLE_BYTES]);
 psml_status psml_xport_destroy(psml_xport x);
 /* One symmetric exchange of n device buffers (what every opening round does). */
 psml_status psml_xport_exchange(psml_xport x, int32_t n, const void *const *send, void *const *recv,
                                 const int64_t *bytes, psml_stream stream);
 /* Bytes and exchanges issued through this transport so far (accounting for bench.py). */
 psml_status psml_xport_stats(psml_xport x, int64_t *bytes_sent, int64_t *exchanges);
+
+/* Data-parallel communicator of ONE party over its `size` GPUs (pair k = ranks k
+ * and k + N/2; party i's N/2 GPUs sum their untruncated gradient shares).  Library-owned NCCL
+ * communicator built from a 128-byte unique id (psml_nccl_unique_id on rank 0 of the party,
+ * broadcast by the caller); size 1 needs no id (uid may be NULL) and makes the all-reduce a no-op.
+ * psml_dp_allreduce: in-place sum of n ring words (uint64_t for l = 64, uint32_t for l = 32) over
+ * the party's ranks = addition in Z_{2^l} (ncclSum on unsigned words wraps), stream-ordered and
+ * graph-capturable. */
+typedef struct psml_dp_s *psml_dp;
+psml_status psml_dp_create(const uint8_t uid[128], int32_t rank, int32_t size, psml_dp *out);
+psml_status psml_dp_destroy(psml_dp dp);
+psml_status psml_dp_size(psml_dp dp, int32_t *size);
+psml_status psml_dp_allreduce(psml_dp dp, void *buf, int64_t n, int32_t l, psml_stream stream);
 
 /* Party `party`'s half of one training step (LINREG / LOGREG / MLP / CNN): X_i: batch x d_0
  * (CNN: batch x C*H*W), Y_i: batch x d_L, this party's shares (device).  The model's dealer
@@ -369,6 +405,17 @@ psml_status psml_party_forward_backward(psml_model model, int32_t party, psml_xp
                                         psml_stream stream);
 psml_status psml_party_apply_update(psml_model model, int32_t party, int32_t extra_shift,
                                     psml_stream stream);
+/* The whole step of one party: psml_party_forward_backward, then psml_dp_allreduce of this
+ * party's gradient share over `dp` (nullable = one pair), then psml_party_apply_update with
+ * extra_shift = log2(dp size) (the size must be a power of two). */
+psml_status psml_party_train_step(psml_model model, int32_t party, psml_xport x, psml_dp dp, const void *X_i,
+                                  const void *Y_i, uint32_t step_id, psml_stream stream);
+/* CUDA-graph capture of psml_party_train_step (same flags as psml_model_capture_step: bit 0 the
+ * dealer in the graph, bit 1 the update (and the all-reduce), bit 2 pipelined dealer); replay with
+ * psml_model_step_graph.  The transport must be graph-capturable (peer memory or NCCL, not a host
+ * callback: PSML_ERR_UNSUPPORTED).  Both parties capture and replay the same step sequence. */
+psml_status psml_party_capture_step(psml_model model, int32_t party, psml_xport x, psml_dp dp, const void *X_i,
+                                    const void *Y_i, int32_t flags, psml_stream stream);
 
 #ifdef __cplusplus
 }

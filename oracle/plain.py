@@ -12,7 +12,6 @@ only differences from the secure run are fixed-point rounding and truncation noi
 """
 import numpy as np
 
-from . import core
 from .protocol import F, LR_SHIFT, MASTER, CNN_GEOM
 
 
@@ -23,6 +22,31 @@ def q(x, f):
 
 def eq9(x):
     return np.clip(x + 0.5, 0.0, 1.0)
+
+
+def conv2d(X4, W, k):
+    """Direct valid stride-1 convolution (cross-correlation), written from its definition and
+    independent of core.im2col:  out[b, oy, ox, o] = sum_{c,ky,kx} X[b, c, oy+ky, ox+kx] *
+    W[(c, ky, kx), o].  X4: (B, C, H, W); W: (C*k*k, Cout) with rows ordered (c, ky, kx)."""
+    B, C, H, Wd = X4.shape
+    OH, OW = H - k + 1, Wd - k + 1
+    Wr = W.reshape(C, k, k, -1)
+    out = np.zeros((B, OH, OW, W.shape[1]), dtype=np.result_type(X4, W))
+    for ky in range(k):
+        for kx in range(k):
+            out += np.einsum("bchw,co->bhwo", X4[:, :, ky:ky + OH, kx:kx + OW], Wr[:, ky, kx, :])
+    return out
+
+
+def conv2d_grad_w(X4, D, k):
+    """dL/dW of conv2d: g[(c, ky, kx), o] = sum_{b,oy,ox} X[b, c, oy+ky, ox+kx] * D[b, oy, ox, o]."""
+    B, C, H, Wd = X4.shape
+    OH, OW = H - k + 1, Wd - k + 1
+    g = np.zeros((C, k, k, D.shape[-1]), dtype=np.result_type(X4, D))
+    for ky in range(k):
+        for kx in range(k):
+            g[:, ky, kx, :] = np.einsum("bchw,bhwo->co", X4[:, :, ky:ky + OH, kx:kx + OW], D)
+    return g.reshape(C * k * k, -1)
 
 
 class PlainModel:
@@ -46,14 +70,14 @@ class PlainModel:
         if self.task == "cnn":
             g = CNN_GEOM
             B = X.shape[0]
-            P = core.im2col(X, g["C"], g["H"], g["W"], g["k"])
-            zc = P @ self.W[0]
+            X4 = X.reshape(B, g["C"], g["H"], g["W"])
+            zc = conv2d(X4, self.W[0], g["k"])               # (B, OH, OW, Cout)
             m0 = zc >= 0
-            h1 = np.maximum(zc, 0.0).reshape(B, -1)
+            h1 = np.maximum(zc, 0.0).reshape(B, -1)          # rows (b), cols (oy, ox, o)
             z2 = h1 @ self.W[1]
             m1 = z2 >= 0
             h2 = np.maximum(z2, 0.0)
-            return [P, h1, h2], [m0.reshape(B, -1), m1], eq9(h2 @ self.W[2])
+            return [X4, h1, h2], [m0.reshape(B, -1), m1], eq9(h2 @ self.W[2])
         raise ValueError(self.task)
 
     def step(self, X, Y):
@@ -66,7 +90,9 @@ class PlainModel:
             a = acts[layer]
             if self.task == "cnn" and layer == 0:
                 g = CNN_GEOM
-                delta = delta.reshape(-1, g["Cout"])
+                OH, OW = g["H"] - g["k"] + 1, g["W"] - g["k"] + 1
+                grads[0] = conv2d_grad_w(a, delta.reshape(-1, OH, OW, g["Cout"]), g["k"])
+                continue
             grads[layer] = a.T @ delta
             if layer > 0:
                 delta = (delta @ self.W[layer].T) * masks[layer - 1]

@@ -151,6 +151,11 @@ struct psml_model_s {
     int deal_pending_pool = -1;        // capture in progress: dealer branch not forked yet
     int deal_after = 0, deal_stage = 0;
     bool deal_alone = false;           // dealer being captured after the online chain (full PRG grid)
+    // split deployment capture (psml_party_capture_step): the party, its pair transport and its
+    // data-parallel communicator; cap_party < 0 = the co-resident engine
+    int cap_party = -1;
+    psml_xport cap_xport = nullptr;
+    psml_dp cap_dp = nullptr;
 };
 
 namespace psml {
@@ -1343,6 +1348,7 @@ psml_status psml_train_forward_backward(psml_model m, const void *const X[2], co
     cudaStream_t s = (cudaStream_t)stream;
     m->pool = pool;
     PSML_TRY(forward_backward(m, (const T *const *)X, (const T *const *)Y, s));
+    m->dealt_step[pool] = -1;   // the step's material is single-use
     m->grads_ready = true;
     return PSML_OK;
 }
@@ -1406,6 +1412,26 @@ psml_status psml_secure_train_step(psml_model m, const void *const X[2], const v
     return psml_train_apply_update(m, 0, stream);
 }
 
+// log2 of a data-parallel group size (the update's extra truncation bits); sizes must be 2^k
+static std::pair<psml_status, int> dp_shift(psml_dp dp) {
+    int32_t n = 1;
+    if (dp && psml_dp_size(dp, &n) != PSML_OK) return {PSML_ERR_INVALID, 0};
+    int sh = 0;
+    while ((1 << sh) < n) ++sh;
+    if ((1 << sh) != n) return {fail(PSML_ERR_INVALID, "data-parallel group size must be a power of two"), 0};
+    return {PSML_OK, sh};
+}
+
+// split deployment: all-reduce this party's untruncated gradient share over its data-parallel
+// group, then update its master / forward weight shares
+static psml_status party_reduce_update(psml_model_s *m, int party, psml_dp dp, cudaStream_t s) {
+    auto sh = dp_shift(dp);
+    PSML_TRY(sh.first);
+    if (dp && sh.second > 0)
+        PSML_TRY(psml_dp_allreduce(dp, m->grad_base + (int64_t)party * m->grad_words, m->grad_words, 64, (psml_stream)s));
+    return psml_party_apply_update(m, party, sh.second, (psml_stream)s);
+}
+
 // One captured step for online pool `pool`.  Non-pipelined: [dealer(pool)] -> online -> [update].
 // Pipelined: online(pool) -> [update] on `s`, concurrently dealer(1 - pool) for the NEXT step on the
 // side stream (fork/join inside the capture), reading the step word = step + 1.
@@ -1439,7 +1465,7 @@ static psml_status capture_one(psml_model_s *m, int pool, const T *const X[2], c
         }
         // models without the fused step (the CNN) run large kernels that fill the GPU: their
         // dealer forks at the start of the step (measured: 51.6K vs 49.4K samples/s forked after)
-        m->deal_after = fused_eligible(m) ? after : 0;
+        m->deal_after = (fused_eligible(m) && m->cap_party < 0) ? after : 0;
         m->deal_stage = 0;
         if (st == PSML_OK && m->deal_after == 0) {
             st = deal_pool(m, 1 - pool, 0, false, m->side, deal_s2(m));
@@ -1452,12 +1478,20 @@ static psml_status capture_one(psml_model_s *m, int pool, const T *const X[2], c
         st = deal_pool(m, pool, 0, false, s);
     }
     m->pool = pool;
-    if (st == PSML_OK) st = forward_backward(m, X, Y, on);
+    const int pp = m->cap_party;
+    if (st == PSML_OK) {
+        if (pp >= 0) {
+            PartyRun r{m, pp, m->cap_xport, on};
+            st = party_forward_backward(r, X[pp], Y[pp]);
+        } else {
+            st = forward_backward(m, X, Y, on);
+        }
+    }
     if (st == PSML_OK) st = deal_fork_point(m, on, true);   // not forked yet: fork here
     m->deal_pending_pool = -1;
     if (st == PSML_OK && (flags & 2)) {
         m->grads_ready = true;
-        st = psml_train_apply_update(m, 0, (psml_stream)on);
+        st = pp >= 0 ? party_reduce_update(m, pp, m->cap_dp, on) : psml_train_apply_update(m, 0, (psml_stream)on);
     }
     if (prio && st == PSML_OK &&
         (cudaEventRecord(m->ev_hi, m->hi) != cudaSuccess || cudaStreamWaitEvent(s, m->ev_hi, 0) != cudaSuccess))
@@ -1487,11 +1521,10 @@ static psml_status capture_one(psml_model_s *m, int pool, const T *const X[2], c
     return PSML_OK;
 }
 
-psml_status psml_model_capture_step(psml_model m, const void *const X[2], const void *const Y[2], int32_t flags,
-                                   psml_stream stream) {
-    if (!m || !X || !Y) return fail(PSML_ERR_INVALID, "null argument");
-    PSML_TRY(check_ptrs({X[0], X[1], Y[0], Y[1]}));
-    if (flags & ~7) return fail(PSML_ERR_INVALID, "flags: bit 0 dealer, bit 1 update, bit 2 pipelined dealer");
+static psml_status capture_common(psml_model m, const void *const X[2], const void *const Y[2], int32_t flags,
+                                  psml_stream stream) {
+    if (flags & ~15) return fail(PSML_ERR_INVALID, "flags: bit 0 dealer, bit 1 update, bit 2 pipelined dealer, bit 3 reuse");
+    if ((flags & 8) && (flags & 5)) return fail(PSML_ERR_INVALID, "flag bit 3 (material reuse) only applies without a dealer");
     cudaStream_t s = (cudaStream_t)stream;
     if (s == nullptr) return fail(PSML_ERR_INVALID, "capture needs a non-default stream");
     for (int g = 0; g < 2; ++g)
@@ -1501,15 +1534,45 @@ psml_status psml_model_capture_step(psml_model m, const void *const X[2], const 
         }
     const int prof = g_prof_cls.exchange(-1);   // no profiling events inside the graphs
     psml_status st = PSML_OK;
-    const int ngraphs = (flags & 4) ? 2 : 1;
+    // one graph per dealer pool, except when the graph deals its own pool 0 (flags bit 0 only)
+    // or replays one pool on purpose (bit 3, benchmark-only material reuse)
+    const bool per_pool = (flags & 4) || !(flags & 9);
+    const int ngraphs = per_pool ? 2 : 1;
     for (int g = 0; g < ngraphs && st == PSML_OK; ++g)
-        st = capture_one(m, (flags & 4) ? g : 0, (const T *const *)X, (const T *const *)Y, flags, s, &m->graph[g],
+        st = capture_one(m, per_pool ? g : 0, (const T *const *)X, (const T *const *)Y, flags, s, &m->graph[g],
                          &m->graph_kernels);
     g_prof_cls.store(prof);
     if (st != PSML_OK) return st;
     m->graph_flags = flags;
     for (int i = 0; i < 2; ++i) { m->cap_X[i] = X[i]; m->cap_Y[i] = Y[i]; }
     return PSML_OK;
+}
+
+psml_status psml_model_capture_step(psml_model m, const void *const X[2], const void *const Y[2], int32_t flags,
+                                   psml_stream stream) {
+    if (!m || !X || !Y) return fail(PSML_ERR_INVALID, "null argument");
+    PSML_TRY(check_ptrs({X[0], X[1], Y[0], Y[1]}));
+    m->cap_party = -1;
+    m->cap_xport = nullptr;
+    m->cap_dp = nullptr;
+    return capture_common(m, X, Y, flags, stream);
+}
+
+psml_status psml_party_capture_step(psml_model m, int32_t party, psml_xport x, psml_dp dp, const void *X_i,
+                                    const void *Y_i, int32_t flags, psml_stream stream) {
+    if (!m || !x) return fail(PSML_ERR_INVALID, "null model or transport");
+    if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
+    PSML_TRY(check_ptrs({X_i, Y_i}));
+    if (dp) PSML_TRY(dp_shift(dp).first);
+    const void *X[2] = {nullptr, nullptr}, *Y[2] = {nullptr, nullptr};
+    X[party] = X_i;
+    Y[party] = Y_i;
+    m->cap_party = party;
+    m->cap_xport = x;
+    m->cap_dp = dp;
+    const psml_status st = capture_common(m, X, Y, flags, stream);
+    if (st != PSML_OK) m->cap_party = -1;
+    return st;
 }
 
 // Client encode + share of a whole minibatch in one launch (psml_model_step_host, Z_2^64): ChaCha20
@@ -1639,19 +1702,27 @@ psml_status psml_model_step_graph(psml_model m, uint32_t step_id, psml_stream st
     if (!m->graph[0]) return fail(PSML_ERR_STATE, "no captured step: call psml_model_capture_step first");
     cudaStream_t s = (cudaStream_t)stream;
     const bool pipelined = (m->graph_flags & 4) != 0;
-    const int pool = pipelined ? (int)(step_id & 1) : 0;
-    if (pipelined && (m->dealt_step[pool] != (int64_t)step_id || !m->dealt_full[pool]))
-        return fail(PSML_ERR_STATE, "pipelined graph: psml_model_deal(step_id) must have filled this step's pool");
+    const bool self_dealt = !pipelined && (m->graph_flags & 1);
+    const bool reuse = (m->graph_flags & 8) != 0;   // benchmark-only: replays pool 0 as dealt
+    const int pool = (self_dealt || reuse) ? 0 : (int)(step_id & 1);
+    // A graph without its own dealer consumes material dealt for exactly this step, once: a
+    // Beaver mask opened twice on different values would leak their difference.
+    if (!self_dealt && !reuse && (m->dealt_step[pool] != (int64_t)step_id || !m->dealt_full[pool]))
+        return fail(PSML_ERR_STATE, "psml_model_deal(step_id) must have filled this step's pool (material is single-use)");
+    if (reuse && (m->dealt_step[0] < 0 || !m->dealt_full[0]))
+        return fail(PSML_ERR_STATE, "reuse graph: pool 0 was never dealt");
     set_word_kernel<<<1, 1, 0, s>>>(m->step_dev, pipelined ? step_id + 1 : step_id);
     PSML_LAUNCH_CHECK();
-    PSML_CUDA_TRY(cudaGraphLaunch(m->graph[pipelined ? pool : 0], s));
+    PSML_CUDA_TRY(cudaGraphLaunch(m->graph[(self_dealt || reuse) ? 0 : pool], s));
     g_launches.fetch_add((uint64_t)m->graph_kernels);   // the graph's kernels are our launches
     if (pipelined) {
+        m->dealt_step[pool] = -1;                        // consumed
         m->dealt_step[1 - pool] = (int64_t)step_id + 1;
         m->dealt_full[1 - pool] = true;
-    } else if (m->graph_flags & 1) {
-        m->dealt_step[0] = step_id;
-        m->dealt_full[0] = true;
+    } else if (self_dealt) {
+        m->dealt_step[0] = -1;
+    } else if (!reuse) {
+        m->dealt_step[pool] = -1;
     }
     m->grads_ready = !(m->graph_flags & 2);
     return PSML_OK;
@@ -1665,7 +1736,9 @@ psml_status psml_secure_infer(psml_model m, const void *const X[2], uint32_t ste
     if (m->dealt_step[pool] != (int64_t)step_id)
         return fail(PSML_ERR_STATE, "psml_model_deal(step_id) must precede inference");
     m->pool = pool;
-    return forward(m, (const T *const *)X, nullptr, (T *const *)Yhat, (cudaStream_t)stream);
+    PSML_TRY(forward(m, (const T *const *)X, nullptr, (T *const *)Yhat, (cudaStream_t)stream));
+    m->dealt_step[pool] = -1;   // the step's material is single-use
+    return PSML_OK;
 }
 
 
@@ -1683,8 +1756,16 @@ psml_status psml_party_forward_backward(psml_model m, int32_t party, psml_xport 
     m->pool = pool;
     PartyRun r{m, party, x, (cudaStream_t)stream};
     PSML_TRY(party_forward_backward(r, (const T *)X_i, (const T *)Y_i));
+    m->dealt_step[pool] = -1;   // the step's material is single-use
     m->grads_ready = true;
     return PSML_OK;
+}
+
+psml_status psml_party_train_step(psml_model m, int32_t party, psml_xport x, psml_dp dp, const void *X_i,
+                                  const void *Y_i, uint32_t step_id, psml_stream stream) {
+    PSML_TRY(psml_party_forward_backward(m, party, x, X_i, Y_i, step_id, stream));
+    if (dp) PSML_TRY(dp_shift(dp).first);
+    return party_reduce_update(m, party, dp, (cudaStream_t)stream);
 }
 
 psml_status psml_party_apply_update(psml_model m, int32_t party, int32_t extra_shift, psml_stream stream) {

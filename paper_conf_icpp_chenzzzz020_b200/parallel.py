@@ -215,17 +215,57 @@ def host_staged_exchange_fn(peer, group=None):
     return fn
 
 
-def make_transport(party, peer, group=None):
-    """NCCL (library-owned communicator; party 0 creates the unique id and sends it to the peer
-    over the process group) when the backend is nccl, else a host-staged callback."""
+def _swap_bytes(blob, party, peer, group=None):
+    """Exchange a small byte blob with the peer rank over the process group (party 0 sends
+    first; device tensors on nccl, host tensors otherwise)."""
+    import torch.distributed as dist
+    dev = "cuda" if dist.get_backend(group) == "nccl" else "cpu"
+    mine = torch.frombuffer(bytearray(blob), dtype=torch.uint8).to(dev)
+    theirs = torch.empty_like(mine)
+    if party == 0:
+        dist.send(mine, peer, group)
+        dist.recv(theirs, peer, group)
+    else:
+        dist.recv(theirs, peer, group)
+        dist.send(mine, peer, group)
+    return bytes(theirs.cpu().numpy().tobytes())
+
+
+def make_transport(party, peer, group=None, kind="peer", capacity_bytes=64 << 20):
+    """The pair transport of the split deployment (include/psml.h):
+      peer      (default) library peer-memory mailboxes mapped over CUDA IPC -- NVLink P2P stores
+                between GPUs, shared HBM for two processes on one GPU; one kernel per exchange,
+                graph-capturable; the process group only ships the 256-byte handles once;
+      nccl      a library-owned 2-rank NCCL communicator (send/recv per exchange);
+      callback  host-staged exchange over the process group (any backend, not capturable)."""
     import torch.distributed as dist
     from . import psml
-    if dist.get_backend(group) == "nccl":
-        uid = torch.zeros(128, dtype=torch.uint8, device="cuda")
-        if party == 0:
-            uid.copy_(torch.frombuffer(bytearray(psml.nccl_unique_id()), dtype=torch.uint8))
-            dist.send(uid, peer, group)
-        else:
-            dist.recv(uid, peer, group)
-        return psml.Transport.nccl(bytes(uid.cpu().numpy().tobytes()), party)
-    return psml.Transport.callback(host_staged_exchange_fn(peer, group))
+    if kind == "peer":
+        xp, blob = psml.Transport.peer(party, capacity_bytes)
+        xp.connect(_swap_bytes(blob, party, peer, group))
+        return xp
+    if kind == "nccl":
+        uid = psml.nccl_unique_id() if party == 0 else bytes(128)
+        got = _swap_bytes(uid, party, peer, group)
+        return psml.Transport.nccl(uid if party == 0 else got, party)
+    if kind == "callback":
+        return psml.Transport.callback(host_staged_exchange_fn(peer, group))
+    raise ValueError(kind)
+
+
+def make_dp(ranks, rank, group=None):
+    """The library-owned data-parallel communicator of one party over its global `ranks`
+    (psml_dp_create): the first rank of the party creates the NCCL unique id and broadcasts it
+    over `group` (a torch.distributed group holding exactly `ranks`)."""
+    import torch.distributed as dist
+    from . import psml
+    size = len(ranks)
+    me = ranks.index(rank)
+    if size == 1:
+        return psml.DataParallel(None, 0, 1)
+    dev = "cuda" if dist.get_backend(group) == "nccl" else "cpu"
+    uid = torch.zeros(128, dtype=torch.uint8, device=dev)
+    if me == 0:
+        uid.copy_(torch.frombuffer(bytearray(psml.nccl_unique_id()), dtype=torch.uint8))
+    dist.broadcast(uid, ranks[0], group)
+    return psml.DataParallel(bytes(uid.cpu().numpy().tobytes()), me, size)

@@ -107,7 +107,16 @@ _SIGS = {
     "psml_xport_stats": (i32, [vp, vp, vp]),
     "psml_party_forward_backward": (i32, [vp, i32, vp, vp, vp, u32, vp]),
     "psml_party_apply_update": (i32, [vp, i32, i32, vp]),
+    "psml_xport_peer_create": (i32, [i32, i64, vp, vp]),
+    "psml_xport_peer_connect": (i32, [vp, vp]),
+    "psml_dp_create": (i32, [vp, i32, i32, vp]),
+    "psml_dp_destroy": (i32, [vp]),
+    "psml_dp_size": (i32, [vp, vp]),
+    "psml_dp_allreduce": (i32, [vp, vp, i64, i32, vp]),
+    "psml_party_train_step": (i32, [vp, i32, vp, vp, vp, vp, u32, vp]),
+    "psml_party_capture_step": (i32, [vp, i32, vp, vp, vp, vp, i32, vp]),
 }
+PEER_HANDLE_BYTES = 256
 EXPORTS = tuple(_SIGS)
 
 _lib = None
@@ -502,10 +511,14 @@ class Model:
     def apply_update(self, extra_shift=0, stream=None):
         _call("psml_train_apply_update", self.handle, extra_shift, _stream(stream))
 
-    def capture_step(self, X, Y, with_deal=True, with_update=True, pipelined=False, stream=None):
+    def capture_step(self, X, Y, with_deal=True, with_update=True, pipelined=False, stream=None,
+                     unsafe_reuse_material=False):
         """Capture one step into a CUDA graph reading the fixed share buffers X, Y (pipelined:
-        the dealer of step s + 1 overlaps the online phase of step s)."""
-        flags = (1 if with_deal else 0) | (2 if with_update else 0) | (4 if pipelined else 0)
+        the dealer of step s + 1 overlaps the online phase of step s).  unsafe_reuse_material
+        (benchmark-only timing of the online phase): replay the material dealt once into pool 0
+        on every step -- never in a real run, reused masks leak."""
+        flags = ((1 if with_deal else 0) | (2 if with_update else 0) | (4 if pipelined else 0)
+                 | (8 if unsafe_reuse_material else 0))
         _call("psml_model_capture_step", self.handle, _pair(X), _pair(Y), flags, _stream(stream))
 
     def graph_nodes(self):
@@ -523,6 +536,18 @@ class Model:
             raise PsmlError("marshal", 1, "step_host: q uint8, y float64 | uint8, yhat_host uint64")
         _call("psml_model_step_host", self.handle, _host_ptr(q), _host_ptr(y), 1 if y.dtype == torch.uint8 else 0,
               share_seed, step, _host_ptr(yhat_host), _stream(stream))
+
+    def party_train_step(self, party, xport, dp, X_i, Y_i, step, stream=None):
+        """Split deployment: forward/backward + this party's gradient all-reduce over `dp`
+        (DataParallel or None) + update (psml_party_train_step)."""
+        _call("psml_party_train_step", self.handle, party, xport.handle, dp.handle if dp else None,
+              _ptr(X_i), _ptr(Y_i), step, _stream(stream))
+
+    def party_capture_step(self, party, xport, dp, X_i, Y_i, with_deal=True, with_update=True,
+                           pipelined=False, stream=None):
+        flags = (1 if with_deal else 0) | (2 if with_update else 0) | (4 if pipelined else 0)
+        _call("psml_party_capture_step", self.handle, party, xport.handle, dp.handle if dp else None,
+              _ptr(X_i), _ptr(Y_i), flags, _stream(stream))
 
     def party_forward_backward(self, party, xport, X_i, Y_i, step, stream=None):
         """Split deployment: party `party`'s half of the step, openings through `xport`."""
@@ -590,6 +615,19 @@ class Transport:
         _call("psml_xport_callback_create", cb, None, ctypes.byref(h))
         return cls(h, keep=cb)
 
+    @classmethod
+    def peer(cls, party, capacity_bytes=64 << 20):
+        """Peer-memory transport (psml_xport_peer_create): returns (transport, handle blob); ship
+        the blob to the peer and call connect() with the peer's blob."""
+        buf = (ctypes.c_uint8 * PEER_HANDLE_BYTES)()
+        h = vp()
+        _call("psml_xport_peer_create", party, capacity_bytes, ctypes.byref(h), ctypes.cast(buf, vp))
+        return cls(h), bytes(buf)
+
+    def connect(self, peer_handle):
+        buf = (ctypes.c_uint8 * PEER_HANDLE_BYTES).from_buffer_copy(peer_handle)
+        _call("psml_xport_peer_connect", self.handle, ctypes.cast(buf, vp))
+
     def stats(self):
         b, n = i64(), i64()
         _call("psml_xport_stats", self.handle, ctypes.byref(b), ctypes.byref(n))
@@ -598,6 +636,37 @@ class Transport:
     def close(self):
         if self.handle:
             lib().psml_xport_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class DataParallel:
+    """psml_dp: one party's library-owned NCCL communicator over its data-parallel GPUs."""
+
+    def __init__(self, uid, rank, size):
+        h = vp()
+        if uid is None:
+            _call("psml_dp_create", None, rank, size, ctypes.byref(h))
+        else:
+            buf = (ctypes.c_uint8 * 128).from_buffer_copy(uid)
+            _call("psml_dp_create", ctypes.cast(buf, vp), rank, size, ctypes.byref(h))
+        self.handle = h
+        self.size = size
+
+    def allreduce_(self, t, stream=None):
+        """In-place Z_{2^l} sum of a contiguous uint64 / uint32 CUDA tensor over the group."""
+        l = 64 if t.dtype in (torch.uint64, torch.int64) else 32
+        _call("psml_dp_allreduce", self.handle, _ptr(t), t.numel(), l, _stream(stream))
+        return t
+
+    def close(self):
+        if self.handle:
+            lib().psml_dp_destroy(self.handle)
             self.handle = None
 
     def __del__(self):

@@ -170,14 +170,17 @@ class SecureTrainer:
 class PartyTrainer(SecureTrainer):
     """One party of the split deployment (Fig. 1b: the two servers in different
     processes / GPUs).  The party holds only its own shares; every opening of the step goes
-    through `transport` (psml.Transport: NCCL over NVLink, or a host-staged callback).
+    through `transport` (psml.Transport: peer memory over NVLink / CUDA IPC, NCCL, or a
+    host-staged callback) and its untruncated gradient share is summed over its data-parallel
+    group by the library-owned communicator `dp` (psml.DataParallel, None = one pair).
     The dealer runs in each party's process and each party reads only its own half of the
     material (the offline phase a deployment ships from the client)."""
 
-    def __init__(self, task, W_init, party, transport, batch=128, pair_id=0, **kw):
+    def __init__(self, task, W_init, party, transport, batch=128, pair_id=0, dp=None, **kw):
         super().__init__(task, W_init, batch=batch, pair_id=pair_id, **kw)
         self.party = party
         self.xport = transport
+        self.dp = dp
 
     def share_batch(self, X, Y, step):
         """Client role: encode + share; this party receives only its own share."""
@@ -185,16 +188,44 @@ class PartyTrainer(SecureTrainer):
         return Xs[self.party], Ys[self.party]
 
     def step_party(self, X_i, Y_i, step, dp_group=None, dp_world=1, deal=True):
-        """Forward/backward with per-round exchanges, [all-reduce of this party's gradient
-        share over the party's data-parallel group], update of this party's weights."""
+        """Forward/backward with per-round exchanges, all-reduce of this party's gradient share
+        over the party's data-parallel group, update of this party's weights.  With a library
+        communicator (self.dp) the whole step is one call (psml_party_train_step); a
+        torch.distributed group (dp_group) is the host-side alternative."""
         if deal:
             self.model.deal(step)
+        if self.dp is not None or dp_world == 1:
+            self.model.party_train_step(self.party, self.xport, self.dp, X_i, Y_i, step)
+            return
         self.model.party_forward_backward(self.party, self.xport, X_i, Y_i, step)
-        if dp_world > 1:
-            ptr, words = self.model.grads()
-            g = _wrap_device_ptr(ptr + 8 * words * self.party, words)
-            ring_allreduce_(g, dp_group)
+        ptr, words = self.model.grads()
+        g = _wrap_device_ptr(ptr + 8 * words * self.party, words)
+        ring_allreduce_(g, dp_group)
         self.model.party_apply_update(self.party, extra_shift=dp_update_shift(dp_world))
+
+    def capture_party(self, pipelined=True):
+        """Capture this party's whole step (dealer [pipelined], online phase with its exchanges,
+        gradient all-reduce, update) into CUDA graph(s) reading fixed share buffers."""
+        d_in = self.model.layer_shape(0)[0] if self.task != "cnn" else 3 * 32 * 32
+        self.Xi = torch.zeros((self.batch, d_in), dtype=torch.uint64, device="cuda")
+        self.Yi = torch.zeros((self.batch, self.out_dim), dtype=torch.uint64, device="cuda")
+        self.gstream = torch.cuda.Stream()
+        self.gstream.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.stream(self.gstream):
+            self.model.party_capture_step(self.party, self.xport, self.dp, self.Xi, self.Yi, with_deal=True,
+                                          with_update=True, pipelined=pipelined, stream=self.gstream)
+        torch.cuda.current_stream().wait_stream(self.gstream)
+        self.pipelined = pipelined
+        self._next_dealt = None
+
+    def graph_step_party(self, X_i, Y_i, step):
+        """Copy this party's shares into the captured buffers and replay the captured step."""
+        self.Xi.copy_(X_i.view(self.Xi.shape), non_blocking=True)
+        self.Yi.copy_(Y_i.view(self.Yi.shape), non_blocking=True)
+        if self.pipelined and self._next_dealt != step:
+            self.model.deal(step)
+        self.model.step_graph(step)
+        self._next_dealt = step + 1
 
     def step(self, X, Y, step):
         X_i, Y_i = self.share_batch(X, Y, step)

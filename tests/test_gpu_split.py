@@ -122,18 +122,19 @@ def test_split_compressed_transmission(tmp_path):
 SPLIT_TASKS = [("linreg", 2), ("logreg", 2), ("mlp", 2), ("cnn", 1)]
 
 
-def _party_train(rank, port, outdir):
+def _party_train(rank, port, outdir, kind):
     import sys
     sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
     import synth
-    from paper_conf_icpp_chenzzzz020_b200.parallel import make_transport
+    from paper_conf_icpp_chenzzzz020_b200.parallel import make_dp, make_transport
     from paper_conf_icpp_chenzzzz020_b200.train import PartyTrainer
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=2)
     torch.cuda.set_device(0)
-    xp = make_transport(rank, 1 - rank)
+    xp = make_transport(rank, 1 - rank, kind=kind)
+    dp = make_dp([rank], rank)          # one pair: the party's data-parallel group is itself
     for task, steps in SPLIT_TASKS:
-        tr = PartyTrainer(task, synth.init_weights(task), rank, xp, backend=1)
+        tr = PartyTrainer(task, synth.init_weights(task), rank, xp, backend=1, dp=dp)
         for s in range(steps):
             X, Y = synth.batch(task, s)
             tr.step(torch.from_numpy(X), torch.from_numpy(Y), s)
@@ -145,14 +146,14 @@ def _party_train(rank, port, outdir):
     sent, n_ex = xp.stats()
     np.save(os.path.join(outdir, f"xstats_{rank}.npy"), np.array([sent, n_ex]))
     xp.close()
+    dp.close()
     dist.destroy_process_group()
 
 
-def test_split_training_matches_oracle(tmp_path):
+def _check_against_oracle(tmp_path, tasks):
     import synth
     from oracle import protocol as OP
-    mp.spawn(_party_train, args=(_free_port(), str(tmp_path)), nprocs=2, join=True)
-    for task, steps in SPLIT_TASKS:
+    for task, steps in tasks:
         om = OP.Model(task, synth.init_weights(task))
         for s in range(steps):
             X, Y = synth.batch(task, s)
@@ -162,5 +163,56 @@ def test_split_training_matches_oracle(tmp_path):
                     got = np.load(tmp_path / f"{task}_s{s}_l{layer}_{p}.npy")
                     assert np.array_equal(got.reshape(om.Wm[layer][p].shape), om.Wm[layer][p]), \
                         (task, s, layer, p)
+
+
+@pytest.mark.parametrize("kind", ["peer", "callback"])
+def test_split_training_matches_oracle(tmp_path, kind):
+    """Two party processes on the one test GPU.  kind=peer: every opening is the library's
+    peer-memory exchange kernel over CUDA-IPC-mapped mailboxes (device to device, no host hop);
+    kind=callback: host-staged gloo.  Each party's master shares equal the oracle's."""
+    mp.spawn(_party_train, args=(_free_port(), str(tmp_path), kind), nprocs=2, join=True)
+    _check_against_oracle(tmp_path, SPLIT_TASKS)
     st = [np.load(tmp_path / f"xstats_{p}.npy") for p in range(2)]
     assert st[0][1] == st[1][1] > 0 and st[0][0] == st[1][0] > 0   # symmetric exchanges
+
+
+GRAPH_TASKS = [("mlp", 4), ("logreg", 3)]
+
+
+def _party_graph(rank, port, outdir):
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import synth
+    from paper_conf_icpp_chenzzzz020_b200.parallel import make_dp, make_transport
+    from paper_conf_icpp_chenzzzz020_b200.train import PartyTrainer
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=2)
+    torch.cuda.set_device(0)
+    xp = make_transport(rank, 1 - rank, kind="peer")
+    dp = make_dp([rank], rank)
+    for task, steps in GRAPH_TASKS:
+        tr = PartyTrainer(task, synth.init_weights(task), rank, xp, dp=dp)
+        X, Y = synth.batch(task, 0)
+        tr.step(torch.from_numpy(X), torch.from_numpy(Y), 0)       # eager first step
+        tr.capture_party(pipelined=True)
+        for s in range(steps):
+            if s > 0:
+                X, Y = synth.batch(task, s)
+                X_i, Y_i = tr.share_batch(X, Y, s)
+                tr.graph_step_party(X_i, Y_i, s)
+            torch.cuda.synchronize()
+            for layer in range(tr.model.n_layers):
+                np.save(os.path.join(outdir, f"{task}_s{s}_l{layer}_{rank}.npy"),
+                        tr.my_master_share(layer).cpu().numpy())
+        tr.close()
+    xp.close()
+    dp.close()
+    dist.destroy_process_group()
+
+
+def test_split_step_cuda_graph_matches_oracle(tmp_path):
+    """The split step captured into a CUDA graph (psml_party_capture_step, pipelined dealer, the
+    peer-memory exchanges and the library data-parallel all-reduce inside the graph) replayed
+    for steps 1..n-1 of two party processes: bit-exact vs the oracle after every step."""
+    mp.spawn(_party_graph, args=(_free_port(), str(tmp_path)), nprocs=2, join=True)
+    _check_against_oracle(tmp_path, GRAPH_TASKS)

@@ -115,3 +115,165 @@ def test_synthetic_batches_are_8bit_pixels():
             assert np.array_equal(Y, y)
     X, _ = synth.batch("mlp", 0)
     assert 0.17 < (X > 0).mean() < 0.21 and X.max() == 1.0 and X[X > 0].min() >= 1 / 255
+
+
+# ---------------------------------------------------------------------------------------------
+# CNN path (config 4; R17): im2col, the conv triplet, the conv Beaver product and the
+# whole CNN step, each pinned against a direct convolution written here from its definition.
+# ---------------------------------------------------------------------------------------------
+def _conv_loops(X4, W, k):
+    """out[b, oy, ox, o] = sum_{c,ky,kx} X[b,c,oy+ky,ox+kx] W[(c,ky,kx), o] by plain loops."""
+    B, C, H, Wd = X4.shape
+    OH, OW, Co = H - k + 1, Wd - k + 1, W.shape[1]
+    out = np.zeros((B, OH, OW, Co), dtype=X4.dtype)
+    with np.errstate(over="ignore"):
+        _conv_loops_into(X4, W, k, out)
+    return out
+
+
+def _conv_loops_into(X4, W, k, out):
+    B, C = X4.shape[:2]
+    _, OH, OW, Co = out.shape
+    for b in range(B):
+        for oy in range(OH):
+            for ox in range(OW):
+                for o in range(Co):
+                    acc = X4.dtype.type(0)
+                    for c in range(C):
+                        for ky in range(k):
+                            for kx in range(k):
+                                acc = acc + X4[b, c, oy + ky, ox + kx] * W[(c * k + ky) * k + kx, o]
+                    out[b, oy, ox, o] = acc
+
+
+def _ring_conv(X4, W, k):
+    """Same definition, vectorised over (b, oy, ox) with uint64 wraparound (mod 2^64)."""
+    B, C, H, Wd = X4.shape
+    OH, OW = H - k + 1, Wd - k + 1
+    out = np.zeros((B, OH, OW, W.shape[1]), dtype=np.uint64)
+    with np.errstate(over="ignore"):
+        for c in range(C):
+            for ky in range(k):
+                for kx in range(k):
+                    win = X4[:, c, ky:ky + OH, kx:kx + OW][..., None]
+                    out += win * W[(c * k + ky) * k + kx][None, None, None, :]
+    return out
+
+
+def _ring_conv_grad_w(X4, D, k):
+    """g[(c,ky,kx), o] = sum_{b,oy,ox} X[b,c,oy+ky,ox+kx] D[b,oy,ox,o] mod 2^64."""
+    B, C, H, Wd = X4.shape
+    OH, OW = H - k + 1, Wd - k + 1
+    g = np.zeros((C * k * k, D.shape[-1]), dtype=np.uint64)
+    with np.errstate(over="ignore"):
+        for c in range(C):
+            for ky in range(k):
+                for kx in range(k):
+                    win = X4[:, c, ky:ky + OH, kx:kx + OW][..., None]
+                    g[(c * k + ky) * k + kx] = (win * D).sum(axis=(0, 1, 2), dtype=np.uint64)
+    return g
+
+
+def test_im2col_matches_direct_convolution(orc):
+    """core.im2col (rows (b, oy, ox), cols (c, ky, kx)) times W equals the convolution loops,
+    exactly in Z_2^64, on a ragged non-square geometry; a transposed window (kx, ky) or a
+    channel-last column order fails it."""
+    C, H, Wd, k, B, Co = 2, 6, 7, 3, 2, 3
+    X = orc.prg(64, 9, orc.tag("cX"), 0, B * C * H * Wd).reshape(B, C * H * Wd)
+    W = orc.prg(64, 9, orc.tag("cW"), 0, C * k * k * Co).reshape(C * k * k, Co)
+    P = orc.im2col(X, C, H, Wd, k)
+    assert P.shape == (B * (H - k + 1) * (Wd - k + 1), C * k * k)
+    got = orc.ring_matmul(P, W).reshape(B, H - k + 1, Wd - k + 1, Co)
+    want = _conv_loops(X.reshape(B, C, H, Wd), W, k)
+    assert np.array_equal(got, want)
+    assert np.array_equal(_ring_conv(X.reshape(B, C, H, Wd), W, k), want)
+
+
+def test_plain_conv_matches_definition():
+    """The fp64 reference's own convolution and its weight gradient (oracle/plain.py, which does
+    not use core.im2col) against the loops and against d<out, D>/dW by finite differences
+    (the objective is linear in W, so the difference quotient is exact up to rounding)."""
+    rng = np.random.default_rng(5)
+    X4 = rng.random((2, 3, 7, 6))
+    W = rng.standard_normal((3 * 9, 4))
+    D = rng.standard_normal((2, 5, 4, 4))
+    out = plain.conv2d(X4, W, 3)
+    assert np.allclose(out, _conv_loops(X4, W, 3), atol=1e-12)
+    g = plain.conv2d_grad_w(X4, D, 3)
+    for (r, o) in ((0, 0), (13, 2), (26, 3)):
+        Wp = W.copy()
+        Wp[r, o] += 1.0
+        fd = (plain.conv2d(X4, Wp, 3) * D).sum() - (out * D).sum()
+        assert abs(fd - g[r, o]) < 1e-9
+
+
+@pytest.mark.parametrize("transpose", [False, True], ids=["fwd_op0", "gradw_op1"])
+def test_conv_triplet_and_conv_matmul_reconstruct(orc, transpose):
+    """conv_triplet: Z_0 + Z_1 = conv(U_0 + U_1, V_0 + V_1) (forward, Z = im2col(U).V) or the
+    conv weight-gradient form im2col(U)^T.V; conv_matmul: C_0 + C_1 = the same convolution of
+    the opened-and-reconstructed operands, exactly mod 2^64 (Eqs. 1-6 on the
+    un-expanded input, R17), for the full CIFAR geometry at 2 images."""
+    g = P.CNN_GEOM
+    B, k = 2, g["k"]
+    OH = g["H"] - k + 1
+    U, V, Z = P.conv_triplet(pair=0, step=3, op=P.OP_GRADW if transpose else P.OP_FWD, B=B,
+                             transpose=transpose)
+    U4 = (U[0] + U[1]).reshape(B, g["C"], g["H"], g["W"])
+    Vs = V[0] + V[1]
+    if transpose:
+        want_Z = _ring_conv_grad_w(U4, Vs.reshape(B, OH, OH, g["Cout"]), k)
+    else:
+        want_Z = _ring_conv(U4, Vs, k).reshape(-1, g["Cout"])
+    assert np.array_equal(Z[0] + Z[1], want_Z)
+    nin = B * g["C"] * g["H"] * g["W"]
+    x = orc.prg(64, 11, orc.tag("cx"), 0, nin).reshape(B, -1)
+    X = orc.share(x, 12, 0)
+    bshape = Vs.shape
+    b = orc.prg(64, 11, orc.tag("cb"), 0, Vs.size).reshape(bshape)
+    Bm = orc.share(b, 12, 1)
+    Bm = (Bm[0].reshape(bshape), Bm[1].reshape(bshape))
+    C0, C1 = P.conv_matmul(X, Bm, U, V, Z, transpose=transpose, trunc=0)
+    x4 = x.reshape(B, g["C"], g["H"], g["W"])
+    want = (_ring_conv_grad_w(x4, b.reshape(B, OH, OH, g["Cout"]), k) if transpose
+            else _ring_conv(x4, b, k).reshape(-1, g["Cout"]))
+    assert np.array_equal(C0 + C1, want)
+
+
+def test_cnn_oracle_step_tracks_fp64():
+    """The whole secure CNN step (oracle/protocol.py _cnn_forward_backward + apply_update) vs the
+    fp64 reference, whose convolution is the direct definition above: per-layer weight
+    gradients (26 fractional bits) within fixed-point noise of the fp64 gradients, predictions
+    within a few LSB, and decoded master weights after 2 steps within 2^-14 (16-image batches to
+    keep the CPU suite short; the one-epoch 2^-12 bar runs on the GPU path)."""
+    task, rows = "cnn", 16
+    Wi = synth.init_weights(task)
+    m, pm = P.Model(task, Wi), plain.PlainModel(task, Wi)
+    from oracle import core
+    for s in range(2):
+        X, Y = synth.batch(task, s)
+        X, Y = X[:rows], Y[:rows]
+        Xs, Ys = P.share_batch(X, Y, s)
+        grads, yhat = P.forward_backward(m, Xs, Ys, s)
+        if s == 0:
+            # fp64 gradients of the same step, from the same forward weights
+            pw = plain.PlainModel(task, Wi)
+            pw.W = [core.decode(core.reconstruct(*w)) for w in m.W]
+            Xq, Yq = plain.q(X, P.F), plain.q(Y, P.F)
+            acts, masks, yh = pw.forward(Xq)
+            got_y = core.decode(core.reconstruct(*yhat)).reshape(yh.shape)
+            assert np.abs(got_y - yh).max() < 2.0 ** -9
+            d = yh - Yq
+            want = [None] * 3
+            want[2] = acts[2].T @ d
+            d = (d @ pw.W[2].T) * masks[1]
+            want[1] = acts[1].T @ d
+            d = (d @ pw.W[1].T) * masks[0]
+            want[0] = plain.conv2d_grad_w(acts[0], d.reshape(rows, 28, 28, 16), 5)
+            for layer in range(3):
+                gl = core.decode(core.reconstruct(*grads[layer]), 64, 2 * P.F).reshape(want[layer].shape)
+                scale = max(1.0, np.abs(want[layer]).max())
+                assert np.abs(gl - want[layer]).max() < 2.0 ** -6 * scale, layer
+        P.apply_update(m, grads)
+        pm.step(X, Y)
+    err = max(np.abs(a - b).max() for a, b in zip(m.decoded_master(), pm.W))
+    assert err < 2.0 ** -14, np.log2(err)
