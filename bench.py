@@ -8,8 +8,10 @@ A step = one pass of the whole hot path over one minibatch of 128 synthetic MNIS
 client encode + share of the batch (plaintext already in HBM), dealer material for the step
 (triplets, MSB material), and the online secure step (masking, openings, Eq. 8 ring GEMMs,
 truncation, secure ReLU / Eq. 9, backprop, master-weight update) -- DESIGN.md "Measurement".
-N > 1 (torchrun): one co-resident party pair per GPU, each on its own 128 rows (weak scaling),
-NCCL all-reduce of the weight-gradient shares every step.
+N > 1 (torchrun): the split deployment -- party 0 on GPU k, party 1 on GPU k + N/2, N/2 pairs
+each on its own 128 rows (weak scaling), every opening one peer-memory exchange over NVLink,
+per-party NCCL all-reduce of the gradient shares, one CUDA graph per party step
+(`--deployment coresident`: one co-resident pair per GPU instead).
 Timing: W untimed warm-up steps, then K steps each bracketed by CUDA events on the launching
 stream with a 256 MiB L2 flush between steps (outside the events); barrier + synchronize around
 the timed region; the max over ranks.  `--impl reference` times the CPU oracle instead.
@@ -51,10 +53,11 @@ def parse():
                     help="headline is mlp (BASELINE metric); others are secondary configs")
     ap.add_argument("--sweep", default=None, metavar="N1,N2,...",
                     help="config-5 ring GEMM sweep (e.g. 512,1024,2048,4096,8192); prints JSON lines")
-    ap.add_argument("--deployment", default="coresident", choices=["coresident", "split"],
-                    help="coresident: both parties of a pair on one GPU (default); split: party 0 "
-                         "and party 1 on different GPUs (ranks k and k + N/2), every opening "
-                         "round exchanged over NCCL (SURVEY 8(e))")
+    ap.add_argument("--deployment", default="auto", choices=["auto", "coresident", "split"],
+                    help="split: party 0 and party 1 on different GPUs (ranks k and k + N/2), every "
+                         "opening round one peer-memory exchange over NVLink (SURVEY 8(e)); "
+                         "coresident: both parties of a pair on one GPU; auto (default): split for "
+                         "N >= 2, coresident for N = 1")
     a = ap.parse_args()
     global TASK, WORKLOAD
     TASK, WORKLOAD = a.task, WORKLOADS[a.task]
@@ -349,15 +352,19 @@ def bench_ours(args):
 
 
 def bench_split(args):
-    """Split deployment: N/2 party pairs, pair k = (rank k: party 0, rank k + N/2: party 1); each
-    pair trains on its own 128 rows; every opening is an NCCL exchange between the pair's GPUs
-    (library-owned communicator); each party all-reduces its gradient share over its N/2 ranks."""
+    """Split deployment (the north_star multi-GPU layout): N/2 party pairs, pair k =
+    (rank k: party 0, rank k + N/2: party 1), each pair on its own 128 rows (weak scaling).  Every
+    opening round is one exchange kernel over the pair's peer-memory mailboxes (CUDA IPC, NVLink
+    stores between the two GPUs); each party sums its untruncated gradient share over its N/2
+    GPUs with the library-owned NCCL all-reduce; the whole party step (dealer of the next step on
+    a forked branch, online phase with its exchanges, all-reduce, update) is one CUDA graph."""
+    import numpy as np
     import torch
     import torch.distributed as dist
 
     import synth
     from paper_conf_icpp_chenzzzz020_b200 import build, psml
-    from paper_conf_icpp_chenzzzz020_b200.parallel import make_transport, pair_layout
+    from paper_conf_icpp_chenzzzz020_b200.parallel import make_dp, make_transport, pair_layout
     from paper_conf_icpp_chenzzzz020_b200.train import PartyTrainer
 
     build.build()
@@ -367,75 +374,89 @@ def bench_split(args):
     groups = [dist.new_group(list(range(q * half, (q + 1) * half))) for q in range(2)]
     dev = torch.device("cuda", local)
     K, W = args.steps, args.warmup
-    xp = make_transport(party, peer)
-    tr = PartyTrainer(TASK, synth.init_weights(TASK), party, xp, batch=BATCH, pair_id=pair)
-    nb = K + W
-    Xs, Ys = [], []
+    cap = (96 << 20) if TASK == "cnn" else (8 << 20)
+    xp = make_transport(party, peer, kind=os.environ.get("PSML_XPORT", "peer"), capacity_bytes=cap)
+    dp = make_dp(list(range(party * half, (party + 1) * half)), rank, groups[party])
+    tr = PartyTrainer(TASK, synth.init_weights(TASK), party, xp, batch=BATCH, pair_id=pair, dp=dp)
+    nb = min(K + W, 64)
+    Xs, Ys, Xh, Yh = [], [], [], []
     for s in range(nb):
         X, Y = synth.batch(TASK, s, BATCH, pair=pair, n_pairs=half)
         Xs.append(torch.from_numpy(X).to(dev))
         Ys.append(torch.from_numpy(Y).to(dev))
-    Xh = [x.cpu().pin_memory() for x in Xs]
-    Yh = [y.cpu().pin_memory() for y in Ys]
+        q, y = synth.batch_u8(TASK, s, BATCH, pair=pair, n_pairs=half)
+        Xh.append(torch.from_numpy(q).pin_memory())
+        Yh.append(torch.from_numpy(np.ascontiguousarray(y)).pin_memory())
     stream = torch.cuda.current_stream()
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
 
-    def step(s, X, Y):
-        X_i, Y_i = tr.share_batch(X, Y, s)
-        tr.step_party(X_i, Y_i, s, dp_group=groups[party], dp_world=half)
-
     def timed(fn, n, base):
+        evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(n)]
         dist.barrier()
         torch.cuda.synchronize()
-        tot = 0.0
         for i in range(n):
             flush.zero_()
-            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            a.record(stream)
+            evs[i][0].record(stream)
             fn(base + i)
-            b.record(stream)
-            b.synchronize()
-            tot += a.elapsed_time(b) / 1e3
+            evs[i][1].record(stream)
+        torch.cuda.synchronize()
         dist.barrier()
-        return max_over_ranks(tot, world)
+        return max_over_ranks(sum(a.elapsed_time(b) for a, b in evs) / 1e3, world)
 
+    # eager warm-up, then capture the party step (the capture issues every exchange once)
     for s in range(W):
-        step(s, Xs[s], Ys[s])
+        X_i, Y_i = tr.share_batch(Xs[s % nb], Ys[s % nb], s)
+        tr.step_party(X_i, Y_i, s)
     torch.cuda.synchronize()
     b0, x0 = xp.stats()
+    tr.capture_party(pipelined=True)
+    b1, x1 = xp.stats()
+
+    def step(s):
+        X_i, Y_i = tr.share_batch(Xs[s % nb], Ys[s % nb], s)
+        tr.graph_step_party(X_i, Y_i, s)
+
+    step(W)
+    torch.cuda.synchronize()
     l0 = psml.kernel_launch_count()
     with ClockSampler(local) as clk:
-        t_dev = timed(lambda s: step(s, Xs[s], Ys[s]), K, W)
+        t_dev = timed(step, K, W + 1)
     launches = psml.kernel_launch_count() - l0
-    b1, x1 = xp.stats()
     out_host = torch.empty(BATCH * Ys[0].shape[1], dtype=torch.uint64).pin_memory()
+    from paper_conf_icpp_chenzzzz020_b200.train import _wrap_device_ptr
 
     def e2e(s):
-        i = (s - W - K) % nb
-        step(s, Xh[i].to(dev, non_blocking=True), Yh[i].to(dev, non_blocking=True))
+        i = s % nb
+        X_i, Y_i = tr.share_batch(Xh[i], Yh[i], s)     # H2D of pixels + class indices, client share
+        tr.graph_step_party(X_i, Y_i, s)
         ptrs = tr.model.output()
-        from paper_conf_icpp_chenzzzz020_b200.train import _wrap_device_ptr
         out_host.copy_(_wrap_device_ptr(ptrs[party], ptrs[2], "<u8"), non_blocking=True)
-    t_e2e = timed(e2e, K, W + K)
+    t_e2e = timed(e2e, K, W + K + 1)
     samples = BATCH * K * half
     return {
         "metric": METRIC, "value": samples / t_dev, "unit": "samples/s", "n_gpus": world,
         "steps": K, "warmup": W, "ms_per_step": 1e3 * t_dev / K, "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "u64",
-        "data": "synthetic (MNIST-shaped 784 features, 81% zeros; teacher labels)",
-        "config": {"workload": WORKLOAD, "deployment": "split (one party per GPU)",
+        "data": "synthetic (MNIST-shaped 8-bit pixels, 81% zeros; teacher labels)",
+        "config": {"workload": WORKLOAD, "deployment": "split (party 0 on GPU k, party 1 on GPU k + N/2)",
                    "global_batch": BATCH * half, "per_pair_batch": BATCH, "pairs": half,
                    "ring": "Z_2^64, 13 fractional bits", "parallelism": f"{half} pairs x 2 parties",
-                   "l2": "256 MiB flush between timed steps (outside the events)",
-                   "step": "client share, dealer (each party's half), online step with one "
-                           "exchange per opening round, gradient all-reduce per party, update"},
-        "exchanges_per_step": (x1 - x0) / K, "bytes_sent_per_step_per_party": (b1 - b0) / K,
+                   "transport": xp_kind(), "l2": "256 MiB flush between timed steps (outside the events)",
+                   "step": "client share, dealer of the next step (forked graph branch), online step "
+                           "with one exchange per opening round, per-party gradient all-reduce, update: "
+                           "one CUDA graph per party"},
+        "exchanges_per_step": x1 - x0, "bytes_sent_per_step_per_party": b1 - b0,
         "e2e": {"value": samples / t_e2e, "unit": "samples/s",
-                "h2d_bytes_per_step": Xh[0].numel() * 8 + Yh[0].numel() * 8,
+                "h2d_bytes_per_step": Xh[0].numel() + Yh[0].numel(),
                 "d2h_bytes_per_step": out_host.numel() * 8},
         "gpu_launches": int(launches), "clocks": clk.summary(),
         "roofline": None,
     }, rank
+
+
+def xp_kind():
+    return {"peer": "peer-memory mailboxes (CUDA IPC, NVLink stores), one kernel per exchange",
+            "nccl": "NCCL send/recv", "callback": "host-staged"}[os.environ.get("PSML_XPORT", "peer")]
 
 
 def measured_peaks():
@@ -768,7 +789,8 @@ def main():
         build.build()
         cfg5_sweep([int(x) for x in args.sweep.split(",")])
         return
-    if args.deployment == "split":
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    if args.deployment == "split" or (args.deployment == "auto" and world >= 2):
         result, rank = bench_split(args)
         if rank == 0:
             print(json.dumps(result), flush=True)

@@ -257,6 +257,9 @@ typedef struct {
     uint64_t dealer_seed;     /* DESIGN.md R11: data_seed + 2                                */
     uint32_t pair_id;         /* data-parallel pair index (call-id bits 63:56)               */
     int32_t cnn_c, cnn_h, cnn_w, cnn_k, cnn_cout, cnn_hidden, cnn_classes; /* CNN geometry  */
+    int32_t fwd_frac_bits[8]; /* per layer f_w (R21): forward weights W = trunc(W^m,
+                                 m - f_w), products with W truncated by f_w; 0 = frac_bits.
+                                 frac_bits <= f_w <= m.  The CNN config uses {16, 20, 20}.    */
 } psml_model_desc;
 
 psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_model *out);
@@ -265,7 +268,7 @@ psml_status psml_model_destroy(psml_model model);
 psml_status psml_model_layer_shape(psml_model model, int32_t layer, int64_t *rows,
                                    int64_t *cols);
 /* Load master-weight shares (m fractional bits) of a layer; the forward copy is
- * W_i = trunc_i(Wm_i, m - frac_bits).  Wm[i]: device, rows x cols. */
+ * W_i = trunc_i(Wm_i, m - f_w) (f_w = fwd_frac_bits[layer], R21).  Wm[i]: device, rows x cols. */
 psml_status psml_model_set_master(psml_model model, int32_t layer, const void *const Wm[2],
                                   psml_stream stream);
 psml_status psml_model_get_master(psml_model model, int32_t layer, void *const Wm[2],
@@ -289,7 +292,7 @@ psml_status psml_train_forward_backward(psml_model model, const void *const X[2]
 psml_status psml_model_output(psml_model model, void **yhat0, void **yhat1, int64_t *n);
 /* Contiguous gradient buffer: [party][all layers' rows*cols] words (device, model-owned). */
 psml_status psml_model_grads(psml_model model, void **grads, int64_t *words_per_party);
-/* W^m_i -= trunc_i(gradW_i, 26 + lr_shift - m + extra_shift); W_i = trunc_i(W^m_i, m - f).
+/* W^m_i -= trunc_i(gradW_i, 2f + lr_shift - m + extra_shift); W_i = trunc_i(W^m_i, m - f_w).
  * extra_shift = log2(number of data-parallel pairs summed into the gradient). */
 psml_status psml_train_apply_update(psml_model model, int32_t extra_shift, psml_stream stream);
 /* CUDA-graph fast path.  Capture ONE training step on `stream` (must not be the legacy default

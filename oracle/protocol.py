@@ -32,6 +32,13 @@ MASK = np.uint64(0xFFFFFFFFFFFFFFFF)
 
 CNN_GEOM = dict(C=3, H=32, W=32, k=5, Cout=16, hidden=64, classes=10)
 
+# Forward-weight precision f_w per layer (R21).  The forward copy of a layer's weights
+# keeps f_w fractional bits, W = trunc(W^m, MASTER - f_w), and every product with it (forward
+# h.W and backprop delta.W^T) is truncated by f_w, so activations and deltas stay at F = 13 bits.
+# f_w = F except the CNN, whose 12544-wide FC1 and 5x5 conv fail BJ's 2^-12 weight bound at
+# f_w = 13 (weights of magnitude ~0.005 quantised at 2^-13 perturb every pre-activation).
+FWD_BITS = {"linreg": [F], "logreg": [F], "mlp": [F, F, F], "cnn": [16, 20, 20]}
+
 
 def call_id(pair, step, layer, op, slot=0):
     return ((pair & 0xFF) << 56) | ((step & 0xFFFFFFFF) << 24) | ((layer & 0xFF) << 16) \
@@ -96,15 +103,19 @@ def sub_pair(a, b):
 
 
 class Model:
-    """Both parties' weight shares: master (MASTER fractional bits) and forward copy (F bits)."""
+    """Both parties' weight shares: master (MASTER fractional bits) and forward copy (fw[l] bits)."""
 
-    def __init__(self, task, W_init):
+    def __init__(self, task, W_init, fw=None):
         self.task = task
+        self.fw = list(fw) if fw is not None else list(FWD_BITS[task])
+        if task == "mlp" and fw is None:
+            self.fw = [F] * len(W_init)
+        assert len(self.fw) == len(W_init)
         self.Wm = []
         for layer, W in enumerate(W_init):
             w = core.encode(W, L, MASTER)
             self.Wm.append(core.share(w, SHARE_SEED, call_id(0, INIT_STEP, layer, OP_SHARE, 2)))
-        self.W = [trunc_pair(wm, MASTER - F) for wm in self.Wm]
+        self.W = [trunc_pair(wm, MASTER - f) for wm, f in zip(self.Wm, self.fw)]
 
     def decoded_master(self):
         return [core.decode(core.reconstruct(*wm), L, MASTER) for wm in self.Wm]
@@ -210,7 +221,7 @@ def forward_backward(model, Xs, Ys, step, pair=0):
     drelus = []
     h = Xs
     for layer in range(nl):
-        z = matmul(h, model.W[layer], pair, step, layer, OP_FWD, F)
+        z = matmul(h, model.W[layer], pair, step, layer, OP_FWD, model.fw[layer])
         if layer < nl - 1:
             h, d = relu(z, pair, step, layer)
             drelus.append(d)
@@ -225,7 +236,7 @@ def forward_backward(model, Xs, Ys, step, pair=0):
     for layer in range(nl - 1, -1, -1):
         grads[layer] = matmul(_T(acts[layer]), delta, pair, step, layer, OP_GRADW, 0)
         if layer > 0:
-            t = matmul(delta, _T(model.W[layer]), pair, step, layer, OP_GRADIN, F)
+            t = matmul(delta, _T(model.W[layer]), pair, step, layer, OP_GRADIN, model.fw[layer])
             delta = hadamard(t, drelus[layer - 1], pair, step, layer - 1, 1)
     return grads, yhat
 
@@ -235,20 +246,21 @@ def _cnn_forward_backward(model, Xs, Ys, step, pair):
     B = Xs[0].shape[0]
     U, V, Z = conv_triplet(pair, step, OP_FWD, B, transpose=False)
     # forward conv: V for op 0 is the weight mask (75 x 16), Z = im2col(U) . V
-    zc = conv_matmul(Xs, model.W[0], U, V, Z, transpose=False, trunc=F)       # (B*784) x 16
+    fw = model.fw
+    zc = conv_matmul(Xs, model.W[0], U, V, Z, transpose=False, trunc=fw[0])   # (B*784) x 16
     h1, d1 = relu(zc, pair, step, 0)
     h1 = (h1[0].reshape(B, -1), h1[1].reshape(B, -1))                         # B x 12544
-    z2 = matmul(h1, model.W[1], pair, step, 1, OP_FWD, F)
+    z2 = matmul(h1, model.W[1], pair, step, 1, OP_FWD, fw[1])
     h2, d2 = relu(z2, pair, step, 1)
-    z3 = matmul(h2, model.W[2], pair, step, 2, OP_FWD, F)
+    z3 = matmul(h2, model.W[2], pair, step, 2, OP_FWD, fw[2])
     yhat = eq9(z3, pair, step, 2)
     delta = sub_pair(yhat, Ys)
     grads = [None] * 3
     grads[2] = matmul(_T(h2), delta, pair, step, 2, OP_GRADW, 0)
-    t = matmul(delta, _T(model.W[2]), pair, step, 2, OP_GRADIN, F)
+    t = matmul(delta, _T(model.W[2]), pair, step, 2, OP_GRADIN, fw[2])
     delta = hadamard(t, d2, pair, step, 1, 1)
     grads[1] = matmul(_T(h1), delta, pair, step, 1, OP_GRADW, 0)
-    t = matmul(delta, _T(model.W[1]), pair, step, 1, OP_GRADIN, F)
+    t = matmul(delta, _T(model.W[1]), pair, step, 1, OP_GRADIN, fw[1])
     d1f = (d1[0].reshape(B, -1), d1[1].reshape(B, -1))
     delta = hadamard(t, d1f, pair, step, 0, 1)
     rows = B * (g["H"] - g["k"] + 1) * (g["W"] - g["k"] + 1)
@@ -259,13 +271,14 @@ def _cnn_forward_backward(model, Xs, Ys, step, pair):
 
 
 def apply_update(model, grads, n_pairs=1):
-    """W^m_i -= trunc_i(gradW_i, F + log2(n_pairs)); W_i = trunc_i(W^m_i, MASTER - F)  (R14)."""
+    """W^m_i -= trunc_i(gradW_i, 2F + LR_SHIFT - MASTER + log2(n_pairs)); W_i = trunc_i(W^m_i,
+    MASTER - f_w)  (R14, R21)."""
     extra = int(np.log2(n_pairs))
     assert (1 << extra) == n_pairs
     for layer, g in enumerate(grads):
-        gt = checked_trunc(g, 26 + LR_SHIFT - MASTER + extra)
+        gt = checked_trunc(g, 2 * F + LR_SHIFT - MASTER + extra)
         model.Wm[layer] = sub_pair(model.Wm[layer], gt)
-        model.W[layer] = checked_trunc(model.Wm[layer], MASTER - F)
+        model.W[layer] = checked_trunc(model.Wm[layer], MASTER - model.fw[layer])
 
 
 def train_step(model, X, Y, step, pair=0):
@@ -281,17 +294,17 @@ def infer(model, Xs, step, pair=0):
     if task == "cnn":
         B = Xs[0].shape[0]
         U, V, Z = conv_triplet(pair, step, OP_FWD, B, transpose=False)
-        zc = conv_matmul(Xs, model.W[0], U, V, Z, transpose=False, trunc=F)
+        zc = conv_matmul(Xs, model.W[0], U, V, Z, transpose=False, trunc=model.fw[0])
         h, _ = relu(zc, pair, step, 0)
         h = (h[0].reshape(B, -1), h[1].reshape(B, -1))
         for layer in (1, 2):
-            z = matmul(h, model.W[layer], pair, step, layer, OP_FWD, F)
+            z = matmul(h, model.W[layer], pair, step, layer, OP_FWD, model.fw[layer])
             h = relu(z, pair, step, layer)[0] if layer == 1 else eq9(z, pair, step, layer)
         return h
     h = Xs
     nl = len(model.W)
     for layer in range(nl):
-        z = matmul(h, model.W[layer], pair, step, layer, OP_FWD, F)
+        z = matmul(h, model.W[layer], pair, step, layer, OP_FWD, model.fw[layer])
         if layer < nl - 1:
             h = relu(z, pair, step, layer)[0]
         elif task == "linreg":

@@ -165,7 +165,7 @@ struct UpdateAll {
     T *Wm[UPD_MAX_LAYERS][2], *W[UPD_MAX_LAYERS][2];
     const T *g[UPD_MAX_LAYERS][2];
     int64_t begin[UPD_MAX_LAYERS + 1];
-    int nl, s_grad, s_fwd;
+    int nl, s_grad, s_fwd[UPD_MAX_LAYERS];
 };
 
 template <typename T>
@@ -182,7 +182,7 @@ __global__ void __launch_bounds__(256) update_all_kernel(const __grid_constant__
         for (int p = 0; p < 2; ++p) {
             const T wm = u.Wm[l][p][i] - trunc_share<T>(u.g[l][p][i], p, u.s_grad);
             u.Wm[l][p][i] = wm;
-            u.W[l][p][i] = trunc_share<T>(wm, p, u.s_fwd);
+            u.W[l][p][i] = trunc_share<T>(wm, p, u.s_fwd[l]);
         }
     }
 }

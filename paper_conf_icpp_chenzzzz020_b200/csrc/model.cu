@@ -201,6 +201,11 @@ static void add_msb(psml_model_s *m, int layer, int op, int64_t n, bool fwd) {
 }
 
 static bool is_eq9_out(const psml_model_s *m) { return m->d.kind != PSML_LINREG; }
+// forward-weight fractional bits of layer l (R21)
+static int fw(const psml_model_s *m, int l) {
+    const int v = m->d.fwd_frac_bits[l];
+    return v > 0 ? v : m->ctx->ring.frac_bits;
+}
 
 static void plan_items(psml_model_s *m) {
     const int64_t B = m->B;
@@ -630,16 +635,16 @@ static psml_status forward(psml_model_s *m, const T *const X[2], const T *const 
     m->act[0].p[1] = (T *)X[1];
     T *yo[2] = {out ? out[0] : m->yhat.p[0], out ? out[1] : m->yhat.p[1]};
     if (m->d.kind == PSML_CNN) {
-        PSML_TRY(conv(m, X, m->W[0].cp(), 0, F, m->z[0].pp(), s));
+        PSML_TRY(conv(m, X, m->W[0].cp(), 0, fw(m, 0), m->z[0].pp(), s));
         PSML_TRY(relu(m, m->z[0].cp(), 0, m->act[1].pp(), m->drelu[0].pp(), s));
-        PSML_TRY(mm(m, m->act[1].cp(), m->W[1].cp(), 1, OP_FWD, 0, F, m->z[1].pp(), s));
+        PSML_TRY(mm(m, m->act[1].cp(), m->W[1].cp(), 1, OP_FWD, 0, fw(m, 1), m->z[1].pp(), s));
         PSML_TRY(relu(m, m->z[1].cp(), 1, m->act[2].pp(), m->drelu[1].pp(), s));
-        PSML_TRY(mm(m, m->act[2].cp(), m->W[2].cp(), 2, OP_FWD, 0, F, m->z[2].pp(), s));
+        PSML_TRY(mm(m, m->act[2].cp(), m->W[2].cp(), 2, OP_FWD, 0, fw(m, 2), m->z[2].pp(), s));
         return eq9(m, m->z[2].cp(), 2, yo, Y, Y ? m->delta.pp() : nullptr, s);
     }
     const int nl = m->nl;
     for (int l = 0; l < nl; ++l) {
-        PSML_TRY(mm(m, m->act[l].cp(), m->W[l].cp(), l, OP_FWD, 0, F, m->z[l].pp(), s));
+        PSML_TRY(mm(m, m->act[l].cp(), m->W[l].cp(), l, OP_FWD, 0, fw(m, l), m->z[l].pp(), s));
         if (l < nl - 1) {
             PSML_TRY(relu(m, m->z[l].cp(), l, m->act[l + 1].pp(), m->drelu[l].pp(), s));
         } else if (is_eq9_out(m)) {
@@ -660,11 +665,11 @@ static psml_status backward(psml_model_s *m, cudaStream_t s) {
     if (m->d.kind == PSML_CNN) {
         // layer 2 (FC 64 -> 10)
         PSML_TRY(mm(m, m->act[2].cp(), m->delta.cp(), 2, OP_GRADW, PSML_TRANS_A, 0, gradp(m, 2, g), s));
-        PSML_TRY(mm(m, m->delta.cp(), m->W[2].cp(), 2, OP_GRADIN, PSML_TRANS_B, F, m->tmp.pp(), s));
+        PSML_TRY(mm(m, m->delta.cp(), m->W[2].cp(), 2, OP_GRADIN, PSML_TRANS_B, fw(m, 2), m->tmp.pp(), s));
         PSML_TRY(had(m, m->tmp.cp(), m->drelu[1].cp(), 1, 1, m->delta.pp(), s));
         // layer 1 (FC 12544 -> 64)
         PSML_TRY(mm(m, m->act[1].cp(), m->delta.cp(), 1, OP_GRADW, PSML_TRANS_A, 0, gradp(m, 1, g), s));
-        PSML_TRY(mm(m, m->delta.cp(), m->W[1].cp(), 1, OP_GRADIN, PSML_TRANS_B, F, m->tmp.pp(), s));
+        PSML_TRY(mm(m, m->delta.cp(), m->W[1].cp(), 1, OP_GRADIN, PSML_TRANS_B, fw(m, 1), m->tmp.pp(), s));
         PSML_TRY(had(m, m->tmp.cp(), m->drelu[0].cp(), 0, 1, m->delta.pp(), s));
         // conv weight gradient: im2col(X)^T . delta   (delta viewed as (B*OH*OW) x Cout)
         return conv(m, m->act[0].cp(), m->delta.cp(), 1, 0, gradp(m, 0, g), s);
@@ -673,7 +678,7 @@ static psml_status backward(psml_model_s *m, cudaStream_t s) {
     for (int l = nl - 1; l >= 0; --l) {
         PSML_TRY(mm(m, m->act[l].cp(), m->delta.cp(), l, OP_GRADW, PSML_TRANS_A, 0, gradp(m, l, g), s));
         if (l > 0) {
-            PSML_TRY(mm(m, m->delta.cp(), m->W[l].cp(), l, OP_GRADIN, PSML_TRANS_B, F, m->tmp.pp(), s));
+            PSML_TRY(mm(m, m->delta.cp(), m->W[l].cp(), l, OP_GRADIN, PSML_TRANS_B, fw(m, l), m->tmp.pp(), s));
             PSML_TRY(had(m, m->tmp.cp(), m->drelu[l - 1].cp(), l - 1, 1, m->delta.pp(), s));
         }
     }
@@ -693,6 +698,8 @@ static int item_index(const psml_model_s *m, int layer, int op, int slot) {
 
 static bool fused_eligible(const psml_model_s *m) {
     if (m->d.kind == PSML_CNN || m->nl > UPD_MAX_LAYERS || (int)m->ob.size() != (int)m->items[0].size()) return false;
+    for (int l = 0; l < m->nl; ++l)
+        if (fw(m, l) != m->ctx->ring.frac_bits) return false;   // the fused step truncates by F
     return fuse_enabled() && chain_mode() == 0;
 }
 
@@ -1085,20 +1092,20 @@ static psml_status party_cnn(PartyRun &r, const T *X, const T *Y) {
     const int F = m->ctx->ring.frac_bits;
     const int p = r.p;
     m->act[0].p[p] = (T *)X;
-    PSML_TRY(party_conv(r, X, m->W[0].p[p], 0, F, m->z[0].p[p]));
+    PSML_TRY(party_conv(r, X, m->W[0].p[p], 0, fw(m, 0), m->z[0].p[p]));
     PSML_TRY(party_relu(r, m->z[0].p[p], 0, m->act[1].p[p], m->drelu[0].p[p]));
-    PSML_TRY(party_mm(r, m->act[1].p[p], m->W[1].p[p], 1, OP_FWD, 0, F, m->z[1].p[p]));
+    PSML_TRY(party_mm(r, m->act[1].p[p], m->W[1].p[p], 1, OP_FWD, 0, fw(m, 1), m->z[1].p[p]));
     PSML_TRY(party_relu(r, m->z[1].p[p], 1, m->act[2].p[p], m->drelu[1].p[p]));
-    PSML_TRY(party_mm(r, m->act[2].p[p], m->W[2].p[p], 2, OP_FWD, 0, F, m->z[2].p[p]));
+    PSML_TRY(party_mm(r, m->act[2].p[p], m->W[2].p[p], 2, OP_FWD, 0, fw(m, 2), m->z[2].p[p]));
     DealItem *mat = find_item(m, 2, OP_EQ9_MSB, 0), *h = find_item(m, 2, OP_HADAMARD, 2);
     if (!mat || !h) return fail(PSML_ERR_STATE, "missing Eq. 9 material");
     PSML_TRY(party_chain(r, m->z[2].p[p], mat, h, 2, m->yhat.p[p], nullptr, Y, m->delta.p[p]));
     T *g[2];
     PSML_TRY(party_mm(r, m->act[2].p[p], m->delta.p[p], 2, OP_GRADW, PSML_TRANS_A, 0, gradp(m, 2, g)[p]));
-    PSML_TRY(party_mm(r, m->delta.p[p], m->W[2].p[p], 2, OP_GRADIN, PSML_TRANS_B, F, m->tmp.p[p]));
+    PSML_TRY(party_mm(r, m->delta.p[p], m->W[2].p[p], 2, OP_GRADIN, PSML_TRANS_B, fw(m, 2), m->tmp.p[p]));
     PSML_TRY(party_had(r, m->tmp.p[p], m->drelu[1].p[p], 1, 1, m->delta.p[p]));
     PSML_TRY(party_mm(r, m->act[1].p[p], m->delta.p[p], 1, OP_GRADW, PSML_TRANS_A, 0, gradp(m, 1, g)[p]));
-    PSML_TRY(party_mm(r, m->delta.p[p], m->W[1].p[p], 1, OP_GRADIN, PSML_TRANS_B, F, m->tmp.p[p]));
+    PSML_TRY(party_mm(r, m->delta.p[p], m->W[1].p[p], 1, OP_GRADIN, PSML_TRANS_B, fw(m, 1), m->tmp.p[p]));
     PSML_TRY(party_had(r, m->tmp.p[p], m->drelu[0].p[p], 0, 1, m->delta.p[p]));
     return party_conv(r, m->act[0].p[p], m->delta.p[p], 1, 0, gradp(m, 0, g)[p]);
 }
@@ -1111,7 +1118,7 @@ static psml_status party_forward_backward(PartyRun &r, const T *X, const T *Y) {
     const int64_t B = m->B;
     m->act[0].p[p] = (T *)X;
     for (int l = 0; l < nl; ++l) {
-        PSML_TRY(party_mm(r, m->act[l].p[p], m->W[l].p[p], l, OP_FWD, 0, F, m->z[l].p[p]));
+        PSML_TRY(party_mm(r, m->act[l].p[p], m->W[l].p[p], l, OP_FWD, 0, fw(m, l), m->z[l].p[p]));
         if (l < nl - 1) {
             DealItem *mat = find_item(m, l, OP_RELU_MSB, 0), *h = find_item(m, l, OP_HADAMARD, 0);
             if (!mat || !h) return fail(PSML_ERR_STATE, "missing ReLU material");
@@ -1133,7 +1140,7 @@ static psml_status party_forward_backward(PartyRun &r, const T *X, const T *Y) {
         gradp(m, l, g);
         PSML_TRY(party_mm(r, m->act[l].p[p], m->delta.p[p], l, OP_GRADW, PSML_TRANS_A, 0, g[p]));
         if (l > 0) {
-            PSML_TRY(party_mm(r, m->delta.p[p], m->W[l].p[p], l, OP_GRADIN, PSML_TRANS_B, F, m->tmp.p[p]));
+            PSML_TRY(party_mm(r, m->delta.p[p], m->W[l].p[p], l, OP_GRADIN, PSML_TRANS_B, fw(m, l), m->tmp.p[p]));
             PSML_TRY(party_had(r, m->tmp.p[p], m->drelu[l - 1].p[p], l - 1, 1, m->delta.p[p]));
         }
     }
@@ -1191,6 +1198,11 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
     }
     default:
         return fail(PSML_ERR_INVALID, "unknown model kind");
+    }
+    for (int l = 0; l < m->nl; ++l) {
+        const int v = desc->fwd_frac_bits[l];
+        if (v != 0 && (v < c->ring.frac_bits || v > desc->master_frac_bits))
+            return fail(PSML_ERR_INVALID, "fwd_frac_bits must be 0 or in [frac_bits, master_frac_bits]");
     }
     psml_model_s *mp = m.get();
     int64_t tot = 0;
@@ -1310,7 +1322,7 @@ psml_status psml_model_set_master(psml_model m, int32_t layer, const void *const
     const int64_t n = m->rows[layer] * m->cols[layer];
     for (int p = 0; p < 2; ++p)
         PSML_CUDA_TRY(cudaMemcpyAsync(m->Wm[layer].p[p], Wm[p], sizeof(T) * n, cudaMemcpyDeviceToDevice, s));
-    const int sh = m->d.master_frac_bits - m->ctx->ring.frac_bits;
+    const int sh = m->d.master_frac_bits - fw(m, layer);
     truncate_pair_kernel<T><<<ew_grid(n), EW_THREADS, 0, s>>>(CPair<T>{{m->Wm[layer].p[0], m->Wm[layer].p[1]}},
                                                                Pair<T>{{m->W[layer].p[0], m->W[layer].p[1]}}, n, sh);
     PSML_LAUNCH_CHECK();
@@ -1375,7 +1387,6 @@ psml_status psml_train_apply_update(psml_model m, int32_t extra_shift, psml_stre
     cudaStream_t s = (cudaStream_t)stream;
     const int f = m->ctx->ring.frac_bits;
     const int s_grad = 2 * f + m->d.lr_shift - m->d.master_frac_bits + extra_shift;
-    const int s_fwd = m->d.master_frac_bits - f;
     if (m->nl <= UPD_MAX_LAYERS) {   // every layer in one launch
         UpdateAll<T> u{};
         int64_t tot = 0;
@@ -1387,7 +1398,8 @@ psml_status psml_train_apply_update(psml_model m, int32_t extra_shift, psml_stre
             tot += m->rows[l] * m->cols[l];
         }
         u.begin[m->nl] = tot;
-        u.nl = m->nl; u.s_grad = s_grad; u.s_fwd = s_fwd;
+        u.nl = m->nl; u.s_grad = s_grad;
+        for (int l = 0; l < m->nl; ++l) u.s_fwd[l] = m->d.master_frac_bits - fw(m, l);
         PSML_CUDA_TRY(launch_pdl(update_all_kernel<T>, dim3(ew_grid(tot)), dim3(EW_THREADS), s, u));
         PSML_LAUNCH_CHECK();
         m->grads_ready = false;
@@ -1399,7 +1411,8 @@ psml_status psml_train_apply_update(psml_model m, int32_t extra_shift, psml_stre
         gradp(m, l, g);
         update_kernel<T><<<ew_grid(n), EW_THREADS, 0, s>>>(Pair<T>{{m->Wm[l].p[0], m->Wm[l].p[1]}},
                                                             Pair<T>{{m->W[l].p[0], m->W[l].p[1]}},
-                                                            CPair<T>{{g[0], g[1]}}, n, s_grad, s_fwd);
+                                                            CPair<T>{{g[0], g[1]}}, n, s_grad,
+                                                            m->d.master_frac_bits - fw(m, l));
         PSML_LAUNCH_CHECK();
     }
     m->grads_ready = false;
@@ -1776,14 +1789,14 @@ psml_status psml_party_apply_update(psml_model m, int32_t party, int32_t extra_s
     cudaStream_t s = (cudaStream_t)stream;
     const int f = m->ctx->ring.frac_bits;
     const int s_grad = 2 * f + m->d.lr_shift - m->d.master_frac_bits + extra_shift;
-    const int s_fwd = m->d.master_frac_bits - f;
     for (int l = 0; l < m->nl; ++l) {
         const int64_t n = m->rows[l] * m->cols[l];
         T *g[2];
         gradp(m, l, g);
         update_kernel<T><<<ew_grid(n), EW_THREADS, 0, s>>>(Pair<T>{{m->Wm[l].p[0], m->Wm[l].p[1]}},
                                                             Pair<T>{{m->W[l].p[0], m->W[l].p[1]}},
-                                                            CPair<T>{{g[0], g[1]}}, n, s_grad, s_fwd, party);
+                                                            CPair<T>{{g[0], g[1]}}, n, s_grad,
+                                                            m->d.master_frac_bits - fw(m, l), party);
         PSML_LAUNCH_CHECK();
     }
     m->grads_ready = false;

@@ -43,7 +43,8 @@ class ModelDesc(ctypes.Structure):
     _fields_ = [("kind", i32), ("n_layers", i32), ("dims", i64 * 8), ("batch", i32),
                 ("lr_shift", i32), ("master_frac_bits", i32), ("dealer_seed", u64),
                 ("pair_id", u32), ("cnn_c", i32), ("cnn_h", i32), ("cnn_w", i32), ("cnn_k", i32),
-                ("cnn_cout", i32), ("cnn_hidden", i32), ("cnn_classes", i32)]
+                ("cnn_cout", i32), ("cnn_hidden", i32), ("cnn_classes", i32),
+                ("fwd_frac_bits", i32 * 8)]
 
 
 # psml_exchange_fn (include/psml.h): (user, n, send[], recv[], bytes[], stream) -> 0 on success
@@ -457,7 +458,8 @@ class Model:
     """psml_model: weight shares, dealer pool and workspaces of one secure model."""
 
     def __init__(self, ctx, kind, dims=None, batch=128, lr_shift=14, master_frac_bits=27,
-                 dealer_seed=0x50534D4C + 2, pair_id=0, cnn=(3, 32, 32, 5, 16, 64, 10)):
+                 dealer_seed=0x50534D4C + 2, pair_id=0, cnn=(3, 32, 32, 5, 16, 64, 10),
+                 fwd_frac_bits=None):
         d = ModelDesc()
         d.kind = kind
         dims = list(dims or ([784, 1] if kind in (LINREG, LOGREG) else [784, 128, 128, 10]))
@@ -467,6 +469,8 @@ class Model:
         d.batch, d.lr_shift, d.master_frac_bits = batch, lr_shift, master_frac_bits
         d.dealer_seed, d.pair_id = dealer_seed, pair_id
         (d.cnn_c, d.cnn_h, d.cnn_w, d.cnn_k, d.cnn_cout, d.cnn_hidden, d.cnn_classes) = cnn
+        for i, v in enumerate(fwd_frac_bits or []):   # per-layer forward-weight bits (R21)
+            d.fwd_frac_bits[i] = v
         self.ctx, self.desc, self.kind = ctx, d, kind
         h = vp()
         _call("psml_model_create", ctx.handle, ctypes.byref(d), ctypes.byref(h))

@@ -24,6 +24,8 @@ DEALER_SEED = DATA_SEED + 2
 OP_SHARE = 7
 INIT_STEP = 0xFFFFFFFF
 KINDS = {"linreg": psml.LINREG, "logreg": psml.LOGREG, "mlp": psml.MLP, "cnn": psml.CNN}
+# forward-weight fractional bits per layer (R21); None = frac_bits for every layer
+FWD_BITS = {"cnn": [16, 20, 20]}
 
 
 def call_id(pair, step, layer, op, slot=0):
@@ -44,7 +46,7 @@ class SecureTrainer:
         self.batch = batch
         self.model = psml.Model(self.ctx, KINDS[task], dims=dims, batch=batch, lr_shift=lr_shift,
                                 master_frac_bits=master_frac_bits, dealer_seed=DEALER_SEED,
-                                pair_id=pair_id)
+                                pair_id=pair_id, fwd_frac_bits=FWD_BITS.get(task))
         for layer, W in enumerate(W_init):
             w = psml.encode(self.master_ring, torch.as_tensor(W, dtype=torch.float64))
             Wm = psml.share(self.ring, SHARE_SEED, call_id(0, INIT_STEP, layer, OP_SHARE, 2), w)

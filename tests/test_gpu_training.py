@@ -167,12 +167,11 @@ def test_one_epoch_bench_path_bitexact_vs_eager_and_fp64(T, task):
 
 
 def test_cnn_one_epoch_against_fp64(T):
-    """Config 4 (CIFAR-shaped CNN, 390 steps of 128): decoded master weights vs fp64 SGD.
-
-    Measured 2^-10.5, NOT BASELINE's 2^-12 (R20): with f = 13 the 12544-wide FC1's
-    forward weights (|w| <= 0.009) quantise at 2^-13, which perturbs every FC1 pre-activation and
-    therefore the output layer's gradient each step (tools/cnn_drift.py: conv 2^-13.2, FC1
-    2^-12.4, output layer 2^-10.5 after one epoch).  The test pins the measured bound."""
+    """Config 4 (CIFAR-shaped CNN, 390 steps of 128): decoded master weights within BASELINE's
+    2^-12 of fp64 SGD.  Needs the forward-weight precision reading R21: at f_w = 13
+    the 12544-wide FC1's and the conv's forward weights quantise too coarsely (measured 2^-10.5);
+    with f_w = (16, 20, 20) the statistical model (tests/analysis/cnn_precision_sim.py) gives
+    2^-14.0."""
     task = "cnn"
     Wi = synth.init_weights(task)
     tr = T.SecureTrainer(task, Wi, backend=0)
@@ -189,7 +188,7 @@ def test_cnn_one_epoch_against_fp64(T):
     got = [w.cpu().numpy() for w in tr.master_weights()]
     err = max(np.abs(g.reshape(w.shape) - w).max() for g, w in zip(got, pm.W))
     print(f"cnn: one-epoch max |w - w_fp64| = 2^{np.log2(err):.2f}")
-    assert err < 2.0 ** -10
+    assert err < 2.0 ** -12
     tr.close()
 
 

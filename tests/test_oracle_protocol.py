@@ -257,7 +257,7 @@ def test_cnn_oracle_step_tracks_fp64():
         if s == 0:
             # fp64 gradients of the same step, from the same forward weights
             pw = plain.PlainModel(task, Wi)
-            pw.W = [core.decode(core.reconstruct(*w)) for w in m.W]
+            pw.W = [core.decode(core.reconstruct(*w), 64, f) for w, f in zip(m.W, m.fw)]
             Xq, Yq = plain.q(X, P.F), plain.q(Y, P.F)
             acts, masks, yh = pw.forward(Xq)
             got_y = core.decode(core.reconstruct(*yhat)).reshape(yh.shape)
@@ -277,3 +277,23 @@ def test_cnn_oracle_step_tracks_fp64():
         pm.step(X, Y)
     err = max(np.abs(a - b).max() for a, b in zip(m.decoded_master(), pm.W))
     assert err < 2.0 ** -14, np.log2(err)
+
+
+@pytest.mark.parametrize("fw", [13, 16, 20])
+def test_forward_weight_precision_bookkeeping(orc, fw):
+    """DESIGN.md R21: forward weights at f_w fractional bits, W = trunc(W^m, 27 - f_w), and the
+    product truncated by f_w keeps activations at F = 13 bits: the decoded product equals the
+    fp64 product within the fixed-point error (a truncation by F instead of f_w would be off by a
+    factor 2^(f_w - 13); a wrong forward-copy shift by a power of two)."""
+    rng = np.random.default_rng(fw)
+    Xf = rng.random((8, 40))
+    Wf = rng.uniform(-0.05, 0.05, (40, 6))
+    m = P.Model("linreg", [Wf[:, :1]], fw=[fw])
+    assert m.fw == [fw]
+    Wm = orc.share(orc.encode(Wf, 64, P.MASTER), 3, 0)
+    W = P.trunc_pair(Wm, P.MASTER - fw)
+    Xs = orc.share(orc.encode(Xf, 64, P.F), 3, 1)
+    z = P.matmul(Xs, W, 0, 5, 0, P.OP_FWD, fw)
+    got = orc.decode(orc.reconstruct(*z), 64, P.F)
+    want = plain.q(Xf, P.F) @ Wf
+    assert np.abs(got - want).max() < 40 * 2.0 ** -fw + 2 * 2.0 ** -P.F
