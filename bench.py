@@ -177,6 +177,7 @@ def bench_ours(args):
     world, rank, local = dist_setup(args)
     dev = torch.device("cuda", local)
     K, W = args.steps, args.warmup
+    whole = ClockSampler(local).__enter__()   # clocks over the whole GPU-active bench
     tr = SecureTrainer(TASK, synth.init_weights(TASK), batch=BATCH, pair_id=rank)
     # plaintext minibatches resident in HBM (and pinned host copies for the e2e leg)
     nb = K + W
@@ -325,29 +326,41 @@ def bench_ours(args):
         "gpu_launches": int(launches),
         "clocks": clk.summary(),
     }
-    # per-kernel-class time inside the same step (CUDA events on the launching stream)
-    classes = {}
+    # Per-kernel-class device time of the headline step, from CUPTI kernel records (torch.profiler)
+    # of K replays of the same pipelined graph; algorithmic work per launch from the library's
+    # counters over K eager steps (psml_prof: ring MACs for GEMM classes, bytes otherwise).
+    work = {}
     base = 3 * (W + K)
-    for cls, name in ((psml.PROF_GEMM, "ring_gemm_cuda_core"), (psml.PROF_TC, "ring_gemm_tcgen05"),
-                      (psml.PROF_MSB, "msb_relu_eq9_rounds"),
-                      (psml.PROF_HAD, "hadamard_rounds"), (psml.PROF_DEALER, "dealer"),
-                      (psml.PROF_MASK, "beaver_mask")):
+    for cls in (psml.PROF_GEMM, psml.PROF_TC, psml.PROF_MSB, psml.PROF_HAD, psml.PROF_DEALER, psml.PROF_MASK):
         psml.prof_enable(cls)
         psml.prof_read()
         for i in range(K):
-            # a GPU sleep ahead of each step lets the host enqueue the whole step first, so the
-            # per-launch events bracket device time, not host submission gaps
-            torch.cuda._sleep(3_000_000)
             one_step(base + i, Xs[i % nb], Ys[i % nb])
-        ms, n, work = psml.prof_read()
+        _, n, w = psml.prof_read()
         psml.prof_enable(-1)
         base += K
-        classes[name] = {"ms_per_step": ms / K, "share_of_step": (ms / K) / result["ms_per_step"],
-                         "launches_per_step": n / K, "work_per_launch": work / max(n, 1),
-                         "ms_per_launch": ms / max(n, 1)}
+        work[PROF_CLASS[cls]] = (n / K, w / max(n, 1))
+    classes = cupti_classes(lambda s: graph_step(s, Xs[s % nb], Ys[s % nb]), K, base, samples / K,
+                            result["ms_per_step"], work)
+    base += K + 1
     result["kernel_classes"] = classes
-    result["roofline"] = roofline(classes, result["clocks"])
+    mac_peak = mac_peak_tmacs()
+    int8 = int8_peak_tops()
+    result["roofline"] = roofline(classes, mac_peak, int8)
     result["offline"] = offline_figure(classes["dealer"], samples / K)
+    gemm_macs = sum(classes[c]["work_per_launch"] * classes[c]["work_launches_per_step_eager"]
+                    for c in ("ring_gemm_cuda_core", "ring_gemm_tcgen05") if c in classes)
+    step_ops = 36 * 2 * gemm_macs
+    result["step_int8_fraction"] = {
+        "useful_limb_ops_per_step": step_ops,
+        "achieved_tops": step_ops / (result["ms_per_step"] / 1e3) / 1e12, "peak_tops": int8[0],
+        "frac": step_ops / (result["ms_per_step"] / 1e3) / 1e12 / int8[0], "peak_source": int8[1],
+        "note": "every Beaver product of the step (both parties, K' = 2K) counted as 36 useful "
+                "limb-pair MMAs x 2 ops per ring MAC, whichever unit ran it"}
+    whole.__exit__()
+    result["clocks_timed_region"] = result["clocks"]
+    result["clocks"] = whole.summary()
+    result["clocks"]["window"] = "whole bench (warm-up, timed legs, profiling legs)"
     return result, tr, world, rank
 
 
@@ -471,52 +484,105 @@ def committed_traffic(name):
     (the newest profiles/r01*_traffic.json, written by tools/traffic.py), or None."""
     import glob
     try:
-        t = json.load(open(sorted(glob.glob(os.path.join(ROOT, "profiles", "r01*_traffic.json")))[-1]))
+        t = json.load(open(sorted(glob.glob(os.path.join(ROOT, "profiles", "r0*_traffic.json")))[-1]))
         return t[name]["bytes_per_launch_avg"], t["source"]
     except (OSError, ValueError, KeyError, IndexError):
         return None, None
 
 
-def roofline(classes, clocks):
-    """Roofline of the dominant kernel class: the largest ONLINE-phase class of the step (the
-    dealer runs concurrently with the online phase in the pipelined graph), DESIGN.md Sec. 8."""
-    r = _roofline(classes, clocks)
-    r["traffic"], src = committed_traffic(r["class"])
-    if src:
-        r["traffic_unit"], r["traffic_source"] = "bytes per launch", src
-    return r
+PROF_CLASS = {0: "ring_gemm_cuda_core", 1: "ring_gemm_tcgen05", 2: "msb_relu_eq9_rounds", 3: "hadamard_rounds",
+              4: "dealer", 5: "beaver_mask"}
+# kernel name -> class (CUPTI records); the dealer's Z = U V products are dealer work
+KERNEL_CLASS = (("ring_gemm_cl_grouped", "dealer"), ("deal_prg", "dealer"), ("dealer_", "dealer"),
+                ("hadamard_triplet", "dealer"), ("msb_dealer", "dealer"), ("prg_kernel", "dealer"),
+                ("seg_gemm", "ring_gemm_cuda_core"), ("ring_gemm", "ring_gemm_cuda_core"),
+                ("tc_seg", "ring_gemm_tcgen05"), ("tc_ring", "ring_gemm_tcgen05"),
+                ("msb_", "msb_relu_eq9_rounds"), ("had_", "hadamard_rounds"), ("hadamard", "hadamard_rounds"),
+                ("eq9", "hadamard_rounds"), ("open", "beaver_mask"), ("mask", "beaver_mask"),
+                ("update", "update"), ("encode_share", "client_share"), ("client_share", "client_share"))
 
 
-def _roofline(classes, clocks):
-    online = [k for k in classes if k != "dealer"]
+def kernel_class(name):
+    for pat, cls in KERNEL_CLASS:
+        if pat in name:
+            return cls
+    return "other"
+
+
+def cupti_classes(step_fn, K, base, samples_per_step, ms_per_step, work):
+    """Kernel durations from CUPTI (torch.profiler CUDA activity) over K calls of step_fn, summed
+    per class: ms_per_step, launches_per_step, ms_per_launch; work_per_launch from `work`."""
+    import torch
+    from torch.profiler import ProfilerActivity, profile
+    step_fn(base)
+    torch.cuda.synchronize()
+    with profile(activities=[ProfilerActivity.CUDA]) as prof:
+        for i in range(K):
+            step_fn(base + 1 + i)
+        torch.cuda.synchronize()
+    tot, cnt = {}, {}
+    for e in prof.events():
+        dt = getattr(e, "device_time", None)
+        if dt is None:
+            dt = getattr(e, "cuda_time", 0.0)
+        if getattr(e, "device_type", None) is not None and "CUDA" not in str(e.device_type):
+            continue
+        if dt <= 0 or e.name.startswith("Memcpy") or e.name.startswith("Memset") or "elementwise" in e.name \
+                or "fill" in e.name.lower():
+            continue
+        c = kernel_class(e.name)
+        tot[c] = tot.get(c, 0.0) + dt / 1e3
+        cnt[c] = cnt.get(c, 0) + 1
+    out = {}
+    for c in tot:
+        n_step, w = work.get(c, (cnt[c] / K, 0.0))
+        out[c] = {"ms_per_step": tot[c] / K, "share_of_step": tot[c] / K / ms_per_step,
+                  "launches_per_step": cnt[c] / K, "ms_per_launch": tot[c] / cnt[c],
+                  "work_per_launch": w, "work_launches_per_step_eager": n_step,
+                  "source": "CUPTI kernel records (torch.profiler) of the replayed step graph"}
+    online = sum(v["ms_per_step"] for k, v in out.items() if k not in ("dealer", "client_share"))
+    out["_check"] = {"online_class_sum_ms": online, "ms_per_step": ms_per_step,
+                     "online_sum_le_step": online <= ms_per_step * 1.02}
+    return out
+
+
+def mac_peak_tmacs():
+    """Measured CUDA-core ring-MAC throughput (psml_bench_mac_peak, Z_2^64), T ring-MAC/s."""
+    from paper_conf_icpp_chenzzzz020_b200 import psml
+    try:
+        return psml.bench_mac_peak(64) / 1e12, "measured: psml_bench_mac_peak (register-only u64 MAC chains, all SMs)"
+    except Exception as e:   # noqa: BLE001
+        return 148 * 64 / 3 * 1.965e9 / 1e12, f"derived (microbenchmark failed: {e})"
+
+
+def roofline(classes, mac_peak, int8):
+    """Roofline of the dominant kernel: the largest ONLINE-phase class of the step by CUPTI device
+    time (the dealer runs concurrently with the online phase in the pipelined graph)."""
+    online = [k for k in classes if k not in ("dealer", "client_share", "_check", "other", "update")]
     name = max(online, key=lambda k: classes[k]["ms_per_step"])
     c = classes[name]
     sec = c["ms_per_launch"] / 1e3
     mp = measured_peaks()
+    sel = "largest online-phase kernel class by CUPTI device time (dealer overlapped)"
     if name == "ring_gemm_tcgen05":
-        # tensor (INT8): useful limb-MMA ops = 36 limb pairs x 2 ops per ring MAC (DESIGN.md 7)
-        peak, src = int8_peak_tops()
         ach = 36 * 2 * c["work_per_launch"] / sec / 1e12
-        return {"bound": "tensor", "class": name, "kernel": "tc_seg_kernel (tcgen05 kind::i8, in-kernel limb split)",
-                "achieved": ach, "peak": peak, "unit": "TOPS", "frac": ach / peak, "traffic": None,
-                "peak_source": src,
-                "selection": "largest online-phase kernel class (dealer overlapped)"}
-    if name == "ring_gemm_cuda_core":
-        # ALU bound: a Z_2^64 multiply-add is 3 IMAD-pipe ops (IMAD.WIDE.U32 + 2 IMAD); B200:
-        # 148 SMs x 4 SMSPs x 16 lanes/clk at clocks.max.sm 1965 MHz (B300_MICROARCH rt=2)
-        peak = 148 * 64 / 3 * 1.965e9 / 1e12
+        r = {"bound": "tensor", "class": name, "kernel": "tc_seg_kernel (tcgen05 kind::i8, in-kernel limb split)",
+             "achieved": ach, "peak": int8[0], "unit": "TOPS", "frac": ach / int8[0], "peak_source": int8[1]}
+    elif name == "ring_gemm_cuda_core":
         ach = c["work_per_launch"] / sec / 1e12
-        return {"bound": "alu", "class": name, "kernel": "seg_gemm_kernel (CUDA-core two-segment Beaver GEMM)",
-                "achieved": ach, "peak": peak,
-                "unit": "T ring-MAC/s", "frac": ach / peak, "traffic": None,
-                "peak_source": "derived: 148 SM x 64 IMAD/clk / 3 IMAD per u64 MAC x 1965 MHz",
-                "selection": "largest online-phase kernel class (dealer overlapped)"}
-    peak = mp.get("hbm_gbs", 6650.0)
-    ach = c["work_per_launch"] / sec / 1e9
-    return {"bound": "hbm", "class": name, "kernel": name, "achieved": ach, "peak": peak, "unit": "GB/s",
-            "frac": ach / peak, "traffic": None,
-            "peak_source": "measured" if "hbm_gbs" in mp else "fallback",
-            "selection": "largest online-phase kernel class (dealer overlapped)"}
+        r = {"bound": "alu", "class": name, "kernel": "seg_gemm_kernel (CUDA-core two-segment Beaver GEMM)",
+             "achieved": ach, "peak": mac_peak[0], "unit": "T ring-MAC/s", "frac": ach / mac_peak[0],
+             "peak_source": mac_peak[1]}
+    else:
+        peak = mp.get("hbm_gbs", 6650.0)
+        ach = c["work_per_launch"] / sec / 1e9
+        r = {"bound": "hbm", "class": name, "kernel": name, "achieved": ach, "peak": peak, "unit": "GB/s",
+             "frac": ach / peak, "peak_source": "measured" if "hbm_gbs" in mp else "fallback"}
+    r["selection"] = sel
+    r["traffic"], src = committed_traffic(name)
+    if src:
+        r["traffic_unit"], r["traffic_source"] = "bytes per launch", src
+    return r
 
 
 def offline_figure(dealer, samples_per_step):
@@ -528,7 +594,7 @@ def offline_figure(dealer, samples_per_step):
     148 SMs x 64 lanes/clk x 1965 MHz (B300_MICROARCH: alu rt_SMSP = 2).  The class time includes
     the Z = U V products, so the fraction is a lower bound for the PRG kernel."""
     sec = dealer["ms_per_step"] / 1e3
-    blocks = dealer["work_per_launch"] * dealer["launches_per_step"]
+    blocks = dealer["work_per_launch"] * dealer.get("work_launches_per_step_eager", dealer["launches_per_step"])
     peak_blocks = 148 * 64 * 1.965e9 / 640
     return {"ms_per_step": dealer["ms_per_step"], "samples_per_s": samples_per_step / sec,
             "chacha20_blocks_per_step": blocks, "prg_output_GBps": blocks * 64 / sec / 1e9,
@@ -536,12 +602,37 @@ def offline_figure(dealer, samples_per_step):
                                  "unit": "G ChaCha20 blocks/s", "frac_lower_bound": blocks / sec / peak_blocks}}
 
 
+_INT8 = None
+
+
 def int8_peak_tops():
-    """Dense INT8 tensor peak: measured cuBLAS bf16 burst x the nominal INT8/bf16 ratio (2)."""
-    mp = measured_peaks()
-    if "bf16_tflops" in mp:
-        return 2.0 * mp["bf16_tflops"], "measured bf16 burst x nominal int8/bf16 ratio 2"
-    return 2.0 * 1590.0, "fallback bf16 1.59 PF x nominal ratio 2"
+    """Dense INT8 tensor ceiling MEASURED on this GPU: cuBLASLt IMMA via torch._int_mm on 8192^3
+    int8 operands (2 n^3 ops, best of 5, CUDA events); fallback: measured bf16 burst x 2."""
+    global _INT8
+    if _INT8 is not None:
+        return _INT8
+    import torch
+    try:
+        n = 8192
+        a = torch.randint(-128, 127, (n, n), dtype=torch.int8, device="cuda")
+        b = torch.randint(-128, 127, (n, n), dtype=torch.int8, device="cuda").t().contiguous().t()
+        for _ in range(2):
+            torch._int_mm(a, b)
+        best = 1e30
+        for _ in range(5):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            torch._int_mm(a, b)
+            e1.record()
+            torch.cuda.synchronize()
+            best = min(best, e0.elapsed_time(e1))
+        _INT8 = (2.0 * n ** 3 / (best / 1e3) / 1e12, "measured: torch._int_mm (cuBLASLt INT8) 8192^3, best of 5")
+        del a, b
+    except Exception as e:   # noqa: BLE001
+        mp = measured_peaks()
+        bf = mp.get("bf16_tflops", 1590.0)
+        _INT8 = (2.0 * bf, f"measured bf16 burst x nominal int8/bf16 ratio 2 (torch._int_mm failed: {e})")
+    return _INT8
 
 
 def ring_gemm_figure(n=4096, l=64, reps=5):
@@ -701,6 +792,16 @@ def cfg5_sweep(ns):
 
 
 
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
+
+
 def cpu_baseline(budget_s=12.0):
     """The oracle as it stands on this host: whole secure MLP training steps (batch 128)."""
     import oracle
@@ -709,7 +810,8 @@ def cpu_baseline(budget_s=12.0):
     n = max(2, min(60, int(budget_s / max(t1, 1e-3))))
     t, cores = oracle_steps(n, base=10001)
     out = {"value": BATCH * n / t, "unit": "samples/s", "cores": cores, "kind": "oracle",
-           "sample": f"{n} full oracle secure MLP training steps (batch 128) on the host"}
+           "sample": f"{n} full oracle secure MLP training steps (batch 128) on the host",
+           "cpu_model": cpu_model(), "nproc": os.cpu_count()}
     # the same oracle on ONE host thread (nproc and 1 thread), a few steps in a
     # subprocess with OMP_NUM_THREADS=1
     try:
@@ -770,7 +872,7 @@ def bench_reference(args, budget_s=150.0):
         "data": ("synthetic (CIFAR-shaped 3x32x32 8-bit pixels; teacher-CNN labels)" if TASK == "cnn" else
                  "synthetic (MNIST-shaped 8-bit pixels, 81% zeros; teacher labels)"),
         "config": arm_config(world),
-        "cpu_baseline": {"value": v, "unit": "samples/s", "cores": cores, "kind": "oracle",
+        "cpu_baseline": {"value": v, "unit": "samples/s", "cores": cores, "kind": "oracle", "cpu_model": cpu_model(),
                          "sample": f"{n} of the {args.steps} requested steps: full oracle secure training "
                                    f"steps of batch {BATCH} (both parties simulated) on the host"},
         "e2e": {"value": v, "unit": "samples/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},

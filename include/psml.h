@@ -82,6 +82,11 @@ uint64_t psml_kernel_launch_count(void);
  * psml_prof_read synchronizes the device, returns the totals and resets them. */
 psml_status psml_prof_enable(int32_t cls);
 psml_status psml_prof_read(double *total_ms, int64_t *launches, double *work);
+/* Measurement utility (synchronous, not part of the hot path): the device's ring multiply-add
+ * throughput in Z_2^l on CUDA cores, measured with a register-only kernel of independent
+ * acc = acc + a * b chains (l = 64: IMAD.WIDE.U32 + 2 IMAD per MAC, the ring GEMM inner loop;
+ * l = 32: one IMAD) on every SM -- the ALU roofline denominator of the CUDA-core ring GEMMs. */
+psml_status psml_bench_mac_peak(int32_t l, double *ring_macs_per_s);
 
 /* ------------------------------------------------------------------------------------------ */
 /* Context                                                                                     */

@@ -115,6 +115,58 @@ psml_status psml_prof_read(double *total_ms, int64_t *launches, double *work) {
     return PSML_OK;
 }
 
+// Ring multiply-add throughput microbenchmark (the ALU roofline denominator of the CUDA-core ring
+// GEMMs): 8 independent accumulator chains per thread of acc = acc + a * b in
+// Z_2^64 (IMAD.WIDE.U32 + 2 IMAD, the GEMM inner loop's mix) or Z_2^32 (one IMAD).
+template <typename T>
+__global__ void __launch_bounds__(256) mac_peak_kernel(T a0, T b0, int iters, T *out) {
+    T acc[8], a[8];
+    const T b = b0 + (T)threadIdx.x;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) { acc[j] = (T)(blockIdx.x * 8 + j); a[j] = a0 + (T)(j * 0x9E3779B9u) + (T)threadIdx.x; }
+    for (int i = 0; i < iters; ++i) {
+#pragma unroll
+        for (int j = 0; j < 8; ++j) acc[j] = acc[j] + a[j] * b;
+#pragma unroll
+        for (int j = 0; j < 8; ++j) a[j] = acc[j];   // chain through memory-free dependencies
+    }
+    T r = 0;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) r ^= acc[j];
+    if (r == (T)0x1234567) out[0] = r;   // keeps the loop alive
+}
+
+psml_status psml_bench_mac_peak(int32_t l, double *ring_macs_per_s) {
+    if ((l != 32 && l != 64) || !ring_macs_per_s) return fail(PSML_ERR_INVALID, "l must be 32 or 64");
+    int dev = 0, sms = 0;
+    PSML_CUDA_TRY(cudaGetDevice(&dev));
+    PSML_CUDA_TRY(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    void *out = nullptr;
+    PSML_CUDA_TRY(cudaMalloc(&out, 8));
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    const int blocks = sms * 8, iters = 4096;
+    float best = 1e30f;
+    for (int rep = 0; rep < 4; ++rep) {
+        cudaEventRecord(e0);
+        if (l == 64) mac_peak_kernel<uint64_t><<<blocks, 256>>>(0x1234567890ull, 0x9E3779B97F4A7C15ull, iters, (uint64_t *)out);
+        else mac_peak_kernel<uint32_t><<<blocks, 256>>>(0x12345u, 0x9E3779B9u, iters, (uint32_t *)out);
+        cudaEventRecord(e1);
+        cudaEventSynchronize(e1);
+        float ms = 0;
+        cudaEventElapsedTime(&ms, e0, e1);
+        if (rep > 0) best = std::min(best, ms);
+    }
+    const cudaError_t e = cudaGetLastError();
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    cudaFree(out);
+    if (e != cudaSuccess) return fail(PSML_ERR_CUDA, cudaGetErrorString(e));
+    *ring_macs_per_s = (double)blocks * 256 * iters * 8 / (best * 1e-3);
+    return PSML_OK;
+}
+
 psml_status psml_device_info(int32_t *sm_count, int32_t *cc_major, int32_t *cc_minor) {
     int dev = 0, n = 0;
     if (cudaGetDeviceCount(&n) != cudaSuccess || n == 0) {

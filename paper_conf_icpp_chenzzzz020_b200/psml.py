@@ -59,6 +59,7 @@ _SIGS = {
     "psml_kernel_launch_count": (u64, []),
     "psml_prof_enable": (i32, [i32]),
     "psml_prof_read": (i32, [vp, vp, vp]),
+    "psml_bench_mac_peak": (i32, [i32, vp]),
     "psml_ctx_create": (i32, [Ring, i32, vp]),
     "psml_ctx_destroy": (i32, [vp]),
     "psml_prg_fill": (i32, [Ring, u64, u32, u64, u64, i64, vp, vp]),
@@ -207,6 +208,13 @@ def kernel_launch_count():
 
 
 PROF_GEMM, PROF_TC, PROF_MSB, PROF_HAD, PROF_DEALER, PROF_MASK = range(6)
+
+
+def bench_mac_peak(l=64):
+    """Measured ring multiply-add throughput on CUDA cores (psml_bench_mac_peak), ring MACs/s."""
+    v = ctypes.c_double()
+    _call("psml_bench_mac_peak", l, ctypes.byref(v))
+    return v.value
 
 
 def prof_enable(cls):
