@@ -49,6 +49,8 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-ring-gemm", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-classes", action="store_true",
+                    help="skip the CUPTI kernel-class leg (required under ncu: one CUPTI client at a time)")
     ap.add_argument("--task", default="mlp", choices=sorted(WORKLOADS),
                     help="headline is mlp (BASELINE metric); others are secondary configs")
     ap.add_argument("--sweep", default=None, metavar="N1,N2,...",
@@ -340,16 +342,24 @@ def bench_ours(args):
         psml.prof_enable(-1)
         base += K
         work[PROF_CLASS[cls]] = (n / K, w / max(n, 1))
-    classes = cupti_classes(lambda s: graph_step(s, Xs[s % nb], Ys[s % nb]), K, base, samples / K,
-                            result["ms_per_step"], work)
-    base += K + 1
-    result["kernel_classes"] = classes
+    classes = None
+    if not args.no_classes and t_on_graph:
+        tr.model.deal(0)
+        gs = torch.cuda.Stream()
+        gs.wait_stream(stream)
+        with torch.cuda.stream(gs):
+            tr.model.capture_step(tr.Xbuf, tr.Ybuf, with_deal=False, with_update=True, pipelined=False,
+                                  stream=gs, unsafe_reuse_material=True)
+        stream.wait_stream(gs)
+        classes = cupti_classes(lambda i: tr.model.step_graph(0), lambda i: tr.model.deal(base + i), K,
+                                1e3 * t_on_graph / K, work)
     mac_peak = mac_peak_tmacs()
     int8 = int8_peak_tops()
-    result["roofline"] = roofline(classes, mac_peak, int8)
-    result["offline"] = offline_figure(classes["dealer"], samples / K)
-    gemm_macs = sum(classes[c]["work_per_launch"] * classes[c]["work_launches_per_step_eager"]
-                    for c in ("ring_gemm_cuda_core", "ring_gemm_tcgen05") if c in classes)
+    if classes:
+        result["kernel_classes"] = classes
+        result["roofline"] = roofline(classes, mac_peak, int8)
+        result["offline"] = offline_figure(classes["dealer"], samples / K)
+    gemm_macs = sum(w[0] * w[1] for c, w in work.items() if c in ("ring_gemm_cuda_core", "ring_gemm_tcgen05"))
     step_ops = 36 * 2 * gemm_macs
     result["step_int8_fraction"] = {
         "useful_limb_ops_per_step": step_ops,
@@ -480,14 +490,16 @@ def measured_peaks():
 
 
 def committed_traffic(name):
-    """DRAM bytes per launch of kernel class `name` from the committed ncu --set full capture
-    (the newest profiles/r01*_traffic.json, written by tools/traffic.py), or None."""
+    """DRAM bytes per launch of kernel class `name` from the newest committed ncu --set full
+    capture that has it (profiles/r0*_traffic.json, written by tools/traffic.py), or None."""
     import glob
-    try:
-        t = json.load(open(sorted(glob.glob(os.path.join(ROOT, "profiles", "r0*_traffic.json")))[-1]))
-        return t[name]["bytes_per_launch_avg"], t["source"]
-    except (OSError, ValueError, KeyError, IndexError):
-        return None, None
+    for f in sorted(glob.glob(os.path.join(ROOT, "profiles", "r0*_traffic.json")), reverse=True):
+        try:
+            t = json.load(open(f))
+            return t[name]["bytes_per_launch_avg"], t["source"]
+        except (OSError, ValueError, KeyError):
+            continue
+    return None, None
 
 
 PROF_CLASS = {0: "ring_gemm_cuda_core", 1: "ring_gemm_tcgen05", 2: "msb_relu_eq9_rounds", 3: "hadamard_rounds",
@@ -509,40 +521,69 @@ def kernel_class(name):
     return "other"
 
 
-def cupti_classes(step_fn, K, base, samples_per_step, ms_per_step, work):
-    """Kernel durations from CUPTI (torch.profiler CUDA activity) over K calls of step_fn, summed
-    per class: ms_per_step, launches_per_step, ms_per_launch; work_per_launch from `work`."""
+def _kernel_records(fn, n):
+    """CUPTI kernel records (name, start_ns, end_ns) of n calls of fn(i) (torch.profiler)."""
     import torch
     from torch.profiler import ProfilerActivity, profile
-    step_fn(base)
-    torch.cuda.synchronize()
     with profile(activities=[ProfilerActivity.CUDA]) as prof:
-        for i in range(K):
-            step_fn(base + 1 + i)
+        for i in range(n):
+            fn(i)
         torch.cuda.synchronize()
+    recs = []
+    for e in prof.profiler.kineto_results.events():
+        if "cuda" not in str(e.device_type()).lower():
+            continue
+        name = e.name()
+        if name.startswith(("Memcpy", "Memset")) or "elementwise" in name or "Fill" in name:
+            continue
+        t0 = e.start_ns()
+        recs.append((name, t0, t0 + e.duration_ns()))
+    return recs
+
+
+def attribute(recs):
+    """Device time per kernel record with overlaps resolved in favour of the EARLIEST-started
+    active kernel: under programmatic dependent launch a kernel's CTAs start while its
+    predecessor still runs and wait (griddepcontrol.wait) -- that wait is the predecessor's time.
+    The attributed times of a run sum to its busy wall time."""
+    ev = sorted(recs, key=lambda r: r[1])
+    out = [0.0] * len(ev)
+    cover = None   # end of the time already attributed
+    for i, (_, t0, t1) in enumerate(ev):
+        lo = t0 if cover is None else max(t0, cover)
+        if t1 > lo:
+            out[i] = (t1 - lo) / 1e6   # ms
+            cover = t1 if cover is None else max(cover, t1)
+    return [(ev[i][0], out[i]) for i in range(len(ev))]
+
+
+def cupti_classes(step_fn, deal_fn, K, ms_step_online, work):
+    """Per-kernel-class device time: CUPTI kernel records of K replays of the online-phase graph
+    (step_fn) and K dealer calls (deal_fn), each kernel's time attributed by `attribute`;
+    work_per_launch from the library counters (`work`)."""
+    import torch
+    step_fn(-1)
+    torch.cuda.synchronize()
     tot, cnt = {}, {}
-    for e in prof.events():
-        dt = getattr(e, "device_time", None)
-        if dt is None:
-            dt = getattr(e, "cuda_time", 0.0)
-        if getattr(e, "device_type", None) is not None and "CUDA" not in str(e.device_type):
-            continue
-        if dt <= 0 or e.name.startswith("Memcpy") or e.name.startswith("Memset") or "elementwise" in e.name \
-                or "fill" in e.name.lower():
-            continue
-        c = kernel_class(e.name)
-        tot[c] = tot.get(c, 0.0) + dt / 1e3
-        cnt[c] = cnt.get(c, 0) + 1
+    for fn in (step_fn, deal_fn):
+        for name, ms in attribute(_kernel_records(fn, K)):
+            c = kernel_class(name)
+            if fn is deal_fn and c != "dealer":
+                c = "dealer"
+            tot[c] = tot.get(c, 0.0) + ms
+            cnt[c] = cnt.get(c, 0) + 1
     out = {}
     for c in tot:
         n_step, w = work.get(c, (cnt[c] / K, 0.0))
-        out[c] = {"ms_per_step": tot[c] / K, "share_of_step": tot[c] / K / ms_per_step,
+        out[c] = {"ms_per_step": tot[c] / K, "share_of_online_step": tot[c] / K / ms_step_online,
                   "launches_per_step": cnt[c] / K, "ms_per_launch": tot[c] / cnt[c],
                   "work_per_launch": w, "work_launches_per_step_eager": n_step,
-                  "source": "CUPTI kernel records (torch.profiler) of the replayed step graph"}
-    online = sum(v["ms_per_step"] for k, v in out.items() if k not in ("dealer", "client_share"))
-    out["_check"] = {"online_class_sum_ms": online, "ms_per_step": ms_per_step,
-                     "online_sum_le_step": online <= ms_per_step * 1.02}
+                  "source": "CUPTI kernel records (torch.profiler), overlap attributed to the earliest-started "
+                            "kernel (PDL waits belong to the predecessor)"}
+    online = sum(v["ms_per_step"] for k, v in out.items() if k != "dealer")
+    out["_check"] = {"online_class_sum_ms": online, "online_graph_ms_per_step": ms_step_online,
+                     "note": "online classes from the online-phase graph (dealer material replayed); "
+                             "dealer from psml_model_deal calls"}
     return out
 
 
@@ -559,6 +600,7 @@ def roofline(classes, mac_peak, int8):
     """Roofline of the dominant kernel: the largest ONLINE-phase class of the step by CUPTI device
     time (the dealer runs concurrently with the online phase in the pipelined graph)."""
     online = [k for k in classes if k not in ("dealer", "client_share", "_check", "other", "update")]
+    online = [k for k in online if k in PROF_CLASS.values()]
     name = max(online, key=lambda k: classes[k]["ms_per_step"])
     c = classes[name]
     sec = c["ms_per_launch"] / 1e3
@@ -659,13 +701,20 @@ def ring_gemm_figure(n=4096, l=64, reps=5):
     pairs = 36 if l == 64 else 10
     useful = pairs * 2.0 * n ** 3
     ctx.close()
+    traffic, tsrc = None, None
+    if n == 4096:
+        g, tsrc = committed_traffic("ring_gemm_tc_l64" if l == 64 else "ring_gemm_tc_l32")
+        sp, _ = committed_traffic("ring_gemm_limb_split")
+        traffic = (g + sp) if (g and sp) else None
     tops = useful / (ms / 1e3) / 1e12
     peak, src = int8_peak_tops()
     return {"n": n, "l": l, "ms": ms, "useful_limb_tops": tops,
             "frac_of_int8_dense_spec_4500": tops / INT8_DENSE_PEAK_TOPS,
             "roofline": {"bound": "tensor", "kernel": "tc_ring_gemm (tcgen05 kind::i8 limbs)",
                          "achieved": tops, "peak": peak, "unit": "TOPS", "frac": tops / peak,
-                         "traffic": None, "peak_source": src},
+                         "traffic": traffic, "traffic_unit": "bytes per call (limb split + GEMM)",
+                         "traffic_source": tsrc, "algorithmic_bytes": 2 * n * n * (l // 8) + n * n * (l // 8),
+                         "peak_source": src},
             "ring_tmacs": n ** 3 / (ms / 1e3) / 1e12}
 
 

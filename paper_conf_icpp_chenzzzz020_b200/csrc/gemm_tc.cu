@@ -338,242 +338,6 @@ __global__ void __launch_bounds__(128, 1) tc_ring_gemm_kernel(const TcParams<T> 
 }
 
 // ------------------------------------------------------------------------------------------------
-// l = 64, v2: N = 128 per MMA, two shift-group passes over 4 TMEM accumulators of 128 columns.
-//   pass L: shifts 0..3 (10 limb pairs, limbs 0..3)   -> low  = sum_s S_s 2^{8s}        (exact)
-//   pass H: shifts 4..7 (26 limb pairs, limbs 0..7)   -> high = sum_s S_s 2^{8(s-4)} mod 2^32
-//   result = low + high * 2^32 mod 2^64.
-// Each MMA (128 x 128 x 32) reads 8 KB of smem per 64 tensor cycles instead of 6 KB per 32: the
-// v1 kernel was bound by the tensor core's shared-memory read path (ncu: tc smem wavefronts 80%).
-// Warps: 0 = TMA producer, 1 = MMA issuer, 2..5 = epilogue (warp w reads TMEM lanes 32 (w%4)..).
-// The pass-L result is staged in the output (or added to the split-K partial) and the pass-H
-// epilogue completes it; the pass-L drain overlaps the pass-H loads already in flight.
-// ------------------------------------------------------------------------------------------------
-template <int STAGES>
-__global__ void __launch_bounds__(192, 1) tc_ring_gemm64_v2(const TcParams<uint64_t> P) {
-    using T = uint64_t;
-    constexpr int BN = 128, L = 8;
-    extern __shared__ __align__(1024) uint8_t smem[];
-    constexpr int A_BYTES = BM * BK, B_BYTES = BN * BK;
-    constexpr int STAGE_BYTES = L * (A_BYTES + B_BYTES);
-    constexpr uint32_t IDESC = idesc_i8(BM, BN);
-    uint64_t *full = (uint64_t *)(smem + STAGES * STAGE_BYTES);
-    uint64_t *empty = full + STAGES;
-    uint64_t *accf = empty + STAGES;     // accumulators ready (phase 0: pass L, phase 1: pass H)
-    uint64_t *acce = accf + 1;           // pass-L accumulators drained
-    uint32_t *tmem_slot = (uint32_t *)(acce + 1);
-
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int party = P.party_base + blockIdx.z % P.nparty, split = blockIdx.z / P.nparty;
-    const int nb = blockIdx.x, rb = blockIdx.y;
-    const int nkb = P.nkb_lo + P.nkb_hi;
-    const int kb0 = split * P.kb_per_split;
-    const int kb1 = min(kb0 + P.kb_per_split, nkb);
-
-    if (threadIdx.x == 0) {
-        for (int s = 0; s < STAGES; ++s) {
-            mbar_init(smem_u32(&full[s]), 1);
-            mbar_init(smem_u32(&empty[s]), 1);
-        }
-        mbar_init(smem_u32(accf), 1);
-        mbar_init(smem_u32(acce), 128);
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    if (warp == 2) {
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_u32(tmem_slot)));
-        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
-    }
-    tc_fence_before();
-    __syncthreads();
-    tc_fence_after();
-    const uint32_t tmem = *tmem_slot;
-
-    if (warp == 0) {
-        if (lane == 0) {
-            // ---------------- TMA producer: pass L (limbs 0..3), then pass H (limbs 0..7) ----------------
-            int stage = 0;
-            uint32_t phase = 0;
-            for (int pass = 0; pass < 2; ++pass) {
-                const int nl = pass == 0 ? 4 : 8;
-                for (int kb = kb0; kb < kb1; ++kb) {
-                    mbar_wait(smem_u32(&empty[stage]), phase ^ 1);
-                    const uint32_t fb = smem_u32(&full[stage]);
-                    mbar_expect_tx(fb, (uint32_t)(nl * (A_BYTES + B_BYTES)));
-                    const bool lo = kb < P.nkb_lo;
-                    const int kk = lo ? kb : kb - P.nkb_lo;
-                    const int nk = lo ? P.nkb_lo : P.nkb_hi;
-                    const uint8_t *a = (lo ? P.A_lo[party] : P.A_hi[party]) + ((int64_t)rb * nk + kk) * A_BYTES;
-                    const uint8_t *b = (lo ? P.B_lo[party] : P.B_hi[party]) + ((int64_t)nb * nk + kk) * B_BYTES;
-                    const int64_t as = lo ? P.a_stride_lo : P.a_stride_hi, bs = lo ? P.b_stride_lo : P.b_stride_hi;
-                    uint8_t *sa = smem + stage * STAGE_BYTES, *sb = sa + L * A_BYTES;
-                    for (int p = 0; p < nl; ++p) bulk_g2s(smem_u32(sa + p * A_BYTES), a + p * as, A_BYTES, fb);
-                    for (int q = 0; q < nl; ++q) bulk_g2s(smem_u32(sb + q * B_BYTES), b + q * bs, B_BYTES, fb);
-                    if (++stage == STAGES) { stage = 0; phase ^= 1; }
-                }
-            }
-        }
-    } else if (warp == 1) {
-        if (lane == 0) {
-            // ---------------- MMA issuer ----------------
-            int stage = 0;
-            uint32_t phase = 0;
-            for (int pass = 0; pass < 2; ++pass) {
-                if (pass == 1) {
-                    mbar_wait(smem_u32(acce), 0);   // epilogue has drained pass L
-                    tc_fence_after();
-                }
-                for (int kb = kb0; kb < kb1; ++kb) {
-                    mbar_wait(smem_u32(&full[stage]), phase);
-                    tc_fence_after();
-                    const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES), sb = sa + L * A_BYTES;
-                    if (pass == 0) {
-#pragma unroll
-                        for (int p = 0; p < 4; ++p) {
-                            const uint64_t ad = smem_desc(sa + p * A_BYTES, 128, 256);
-#pragma unroll
-                            for (int q = 0; q < 4 - p; ++q)
-                                tc_mma_i8(tmem + (uint32_t)((p + q) * BN), ad, smem_desc(sb + q * B_BYTES, 128, 256),
-                                          IDESC, (kb > kb0 || p > 0) ? 1u : 0u);
-                        }
-                    } else {
-#pragma unroll
-                        for (int p = 0; p < 8; ++p) {
-                            const uint64_t ad = smem_desc(sa + p * A_BYTES, 128, 256);
-#pragma unroll
-                            for (int q = (p < 4 ? 4 - p : 0); q < 8 - p; ++q)
-                                tc_mma_i8(tmem + (uint32_t)((p + q - 4) * BN), ad,
-                                          smem_desc(sb + q * B_BYTES, 128, 256), IDESC, (kb > kb0 || p > 0) ? 1u : 0u);
-                        }
-                    }
-                    tc_commit(smem_u32(&empty[stage]));
-                    if (++stage == STAGES) { stage = 0; phase ^= 1; }
-                }
-                tc_commit(smem_u32(accf));
-            }
-        }
-    } else {
-        // ---------------- epilogue warps 2..5 ----------------
-        // Direct per-row stores: staging through smem here would compete with the tensor core's
-        // smem reads of pass H, which this epilogue overlaps (measured slower).
-        const int quarter = warp & 3;
-        const int64_t row = (int64_t)rb * BM + quarter * 32 + lane;
-        const uint32_t lane_base = tmem + ((uint32_t)(quarter * 32) << 16);
-        const int64_t col0 = (int64_t)nb * BN;
-        // pass L: low = sum_{s<4} S_s 2^{8s}
-        mbar_wait(smem_u32(accf), 0);
-        tc_fence_after();
-#pragma unroll 1
-        for (int j0 = 0; j0 < BN; j0 += 16) {
-            T acc[16];
-#pragma unroll
-            for (int j = 0; j < 16; ++j) acc[j] = 0;
-#pragma unroll
-            for (int s = 0; s < 4; ++s) {
-                uint32_t r[16];
-                tmem_ld16(lane_base + (uint32_t)(s * BN + j0), r);
-#pragma unroll
-                for (int j = 0; j < 16; ++j) acc[j] += (T)r[j] << (8 * s);
-            }
-            if (j0 == BN - 16) {   // TMEM fully read: pass H may start before this last store
-                tc_fence_before();
-                mbar_arrive(smem_u32(acce));
-            }
-            if (row < P.M && !(P.debug & 2)) {
-#pragma unroll
-                for (int j = 0; j < 16; ++j) {
-                    const int64_t col = col0 + j0 + j;
-                    if (col >= P.N) break;
-                    const int64_t o = row * P.N + col;
-                    if (P.mode == 3) atomicAdd((unsigned long long *)(P.partial + (int64_t)(party - P.party_base) * P.M * P.N + o), acc[j]);
-                    else P.C[P.mode == 2 ? 0 : party][o] = acc[j];
-                }
-            }
-        }
-        // pass H: high = sum_{s>=4} S_s 2^{8(s-4)} mod 2^32, result = low + high 2^32.  Direct
-        // per-row read-modify-write: each thread's 16 consecutive words fill whole sectors over
-        // the loop (staging through smem measured slower, tools/tc_sweep.py).
-        mbar_wait(smem_u32(accf), 1);
-        tc_fence_after();
-#pragma unroll 1
-        for (int j0 = 0; j0 < BN; j0 += 16) {
-            uint32_t hi[16];
-#pragma unroll
-            for (int j = 0; j < 16; ++j) hi[j] = 0;
-#pragma unroll
-            for (int s = 0; s < 4; ++s) {
-                uint32_t r[16];
-                tmem_ld16(lane_base + (uint32_t)(s * BN + j0), r);
-#pragma unroll
-                for (int j = 0; j < 16; ++j) hi[j] += r[j] << (8 * s);
-            }
-            if (row < P.M && !(P.debug & 1)) {
-#pragma unroll
-                for (int j = 0; j < 16; ++j) {
-                    const int64_t col = col0 + j0 + j;
-                    if (col >= P.N) break;
-                    const int64_t o = row * P.N + col;
-                    const T h = (T)hi[j] << 32;
-                    switch (P.mode) {
-                    case 0: P.C[party][o] = P.C[party][o] + h; break;
-                    case 1: P.C[party][o] = trunc_share<T>(P.C[party][o] + h + P.Z[party][o], party, P.trunc); break;
-                    case 2: P.C[0][o] = P.C[0][o] + h - P.Z[0][o]; break;
-                    default: atomicAdd((unsigned long long *)(P.partial + (int64_t)(party - P.party_base) * P.M * P.N + o), h);
-                    }
-                }
-            }
-        }
-    }
-    tc_fence_before();
-    __syncthreads();
-    if (warp == 2) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tmem));
-}
-
-// ------------------------------------------------------------------------------------------------
-// l = 64, v3: the v2 two-pass schedule on a CTA PAIR (cluster of 2, tcgen05 cta_group::2).
-// M = 256 per MMA (128 rows in each CTA's TMEM), N = 128: each CTA stages its own 128 A rows and
-// HALF of the B tile (64 rows = one contiguous 2 KB half of the tiled B limb tile), so per SM an
-// MMA reads 6 KB of smem per 64 tensor cycles (v2: 8 KB) and L2 traffic per output drops by 25%.
-// The leader (rank 0) issues every MMA; commits are multicast to both CTAs' barriers.  The peer's
-// "stage landed" is forwarded to the leader's full barrier by a remote mbarrier arrive (1-D bulk
-// copies have no cta_group::2 form).  Pass-L drain: the leader waits for both CTAs' epilogues.
-// ------------------------------------------------------------------------------------------------
-__device__ __forceinline__ uint32_t cluster_rank() {
-    uint32_t r;
-    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
-    return r;
-}
-__device__ __forceinline__ uint32_t map_to_rank(uint32_t addr, uint32_t rank) {
-    uint32_t r;
-    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(addr), "r"(rank));
-    return r;
-}
-__device__ __forceinline__ void mbar_arrive_remote(uint32_t cluster_addr) {
-    asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
-}
-__device__ __forceinline__ void cluster_sync_all() {
-    asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
-}
-__device__ __forceinline__ void tc_mma_i8_2sm(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
-                                              uint32_t accumulate) {
-    asm volatile(
-        "{\n"
-        ".reg .pred p;\n"
-        "setp.ne.b32 p, %4, 0;\n"
-        "tcgen05.mma.cta_group::2.kind::i8 [%0], %1, %2, %3, p;\n"
-        "}\n" ::"r"(d_tmem),
-        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
-        : "memory");
-}
-__device__ __forceinline__ void tc_commit_2sm(uint32_t bar) {
-    asm volatile(
-        "{\n"
-        ".reg .b16 m;\n"
-        "mov.b16 m, 3;\n"
-        "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], m;\n"
-        "}\n" ::"r"(bar)
-        : "memory");
-}
-
-// ------------------------------------------------------------------------------------------------
 // l = 64, v4: v2 with the passes reversed and the high half kept ON CHIP.
 //   pass H first (shifts 4..7, 26 limb pairs): the epilogue warps fold the 4 accumulators into
 //   high = sum S_s 2^{8(s-4)} mod 2^32 and park it in shared memory (128 x 128 x 4 B = 64 KB);
@@ -770,418 +534,6 @@ __global__ void __launch_bounds__(192, 1) tc_ring_gemm64_v4(const TcParams<uint6
 
 constexpr size_t smem_v4_bytes() { return (size_t)2 * 8 * (BM * BK + 128 * BK) + (size_t)BM * 128 * 4 + 16 * 8; }
 
-// ------------------------------------------------------------------------------------------------
-// l = 64, v5: v4 made PERSISTENT (one CTA per SM, static round-robin over (n-tile, m-tile, split,
-// party) work items).  The epilogue releases TMEM right after reading the pass-L accumulators
-// (barrier tfree), so the global stores of tile i overlap the pass-H MMAs of tile i+1, and the
-// producer starts tile i+1's loads as soon as tile i's pass-L slots retire.  Barrier phases run
-// on across tiles: accf completes twice per tile, acce and tfree once.
-// ------------------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(192, 1) tc_ring_gemm64_v5(const TcParams<uint64_t> P, int n_tiles_n, int n_tiles_m,
-                                                           int n_splits) {
-    using T = uint64_t;
-    constexpr int BN = 128, L = 8;
-    constexpr int A_BYTES = BM * BK, B_BYTES = BN * BK;
-    constexpr int REGION = 2 * L * (A_BYTES + B_BYTES);
-    constexpr int SH_BYTES = L * (A_BYTES + B_BYTES), SL_BYTES = 4 * (A_BYTES + B_BYTES);
-    constexpr uint32_t IDESC = idesc_i8(BM, BN);
-    extern __shared__ __align__(1024) uint8_t smem[];
-    uint32_t *hi_buf = (uint32_t *)(smem + REGION);
-    uint64_t *bars = (uint64_t *)(smem + REGION + BM * BN * 4);
-    uint64_t *fullH = bars, *emptyH = bars + 2, *fullL = bars + 4, *emptyL = bars + 8;
-    uint64_t *accf = bars + 12, *acce = bars + 13, *tfree = bars + 14;
-    uint32_t *tmem_slot = (uint32_t *)(bars + 15);
-
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int nkb = P.nkb_lo + P.nkb_hi;
-    const int64_t n_items = (int64_t)n_tiles_n * n_tiles_m * n_splits * P.nparty;
-
-    if (threadIdx.x == 0) {
-        for (int s = 0; s < 2; ++s) { mbar_init(smem_u32(&fullH[s]), 1); mbar_init(smem_u32(&emptyH[s]), 1); }
-        for (int s = 0; s < 4; ++s) { mbar_init(smem_u32(&fullL[s]), 1); mbar_init(smem_u32(&emptyL[s]), 1); }
-        mbar_init(smem_u32(accf), 1);
-        mbar_init(smem_u32(acce), 128);
-        mbar_init(smem_u32(tfree), 128);
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    if (warp == 2) {
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_u32(tmem_slot)));
-        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
-    }
-    tc_fence_before();
-    __syncthreads();
-    tc_fence_after();
-    const uint32_t tmem = *tmem_slot;
-
-    // work item -> (party, split, rb, nb); n fastest so consecutive CTAs share A tiles in L2
-    auto decode = [&](int64_t it, int &party, int &kb0, int &kb1, int &rb, int &nb) {
-        nb = (int)(it % n_tiles_n);
-        int64_t r = it / n_tiles_n;
-        rb = (int)(r % n_tiles_m);
-        r /= n_tiles_m;
-        const int split = (int)(r % n_splits);
-        party = P.party_base + (int)(r / n_splits);
-        kb0 = split * P.kb_per_split;
-        kb1 = min(kb0 + P.kb_per_split, nkb);
-    };
-    auto tile_src = [&](int party, int rb, int nb, int kb, const uint8_t *&a, const uint8_t *&b, int64_t &as,
-                        int64_t &bs) {
-        const bool lo = kb < P.nkb_lo;
-        const int kk = lo ? kb : kb - P.nkb_lo;
-        const int nk = lo ? P.nkb_lo : P.nkb_hi;
-        a = (lo ? P.A_lo[party] : P.A_hi[party]) + ((int64_t)rb * nk + kk) * A_BYTES;
-        b = (lo ? P.B_lo[party] : P.B_hi[party]) + ((int64_t)nb * nk + kk) * B_BYTES;
-        as = lo ? P.a_stride_lo : P.a_stride_hi;
-        bs = lo ? P.b_stride_lo : P.b_stride_hi;
-    };
-
-    if (warp == 0) {
-        if (lane == 0) {
-            int sh = 0, sl = 0;
-            uint32_t phh = 0, phl = 0;
-            for (int64_t it = blockIdx.x; it < n_items; it += gridDim.x) {
-                int party, kb0, kb1, rb, nb;
-                decode(it, party, kb0, kb1, rb, nb);
-                // the pass-H ring overlaps the pass-L ring's region: wait until the most recent
-                // fill of every L slot was released (a peek: the ring counters do not advance)
-                for (int i = 0; i < 4; ++i)
-                    mbar_wait(smem_u32(&emptyL[(sl + i) & 3]), (phl ^ 1) ^ ((sl + i) >= 4 ? 1u : 0u));
-                for (int kb = kb0; kb < kb1; ++kb) {
-                    mbar_wait(smem_u32(&emptyH[sh]), phh ^ 1);
-                    const uint32_t fb = smem_u32(&fullH[sh]);
-                    mbar_expect_tx(fb, (uint32_t)SH_BYTES);
-                    const uint8_t *a, *b;
-                    int64_t as, bs;
-                    tile_src(party, rb, nb, kb, a, b, as, bs);
-                    uint8_t *sa = smem + sh * SH_BYTES, *sb = sa + L * A_BYTES;
-                    for (int q = 0; q < L; ++q) bulk_g2s(smem_u32(sa + q * A_BYTES), a + q * as, A_BYTES, fb);
-                    for (int q = 0; q < L; ++q) bulk_g2s(smem_u32(sb + q * B_BYTES), b + q * bs, B_BYTES, fb);
-                    if (++sh == 2) { sh = 0; phh ^= 1; }
-                }
-                for (int i = 0; i < 2; ++i)   // all H slots released before the L ring reuses them
-                    mbar_wait(smem_u32(&emptyH[(sh + i) & 1]), (phh ^ 1) ^ ((sh + i) >= 2 ? 1u : 0u));
-                for (int kb = kb0; kb < kb1; ++kb) {
-                    mbar_wait(smem_u32(&emptyL[sl]), phl ^ 1);
-                    const uint32_t fb = smem_u32(&fullL[sl]);
-                    mbar_expect_tx(fb, (uint32_t)SL_BYTES);
-                    const uint8_t *a, *b;
-                    int64_t as, bs;
-                    tile_src(party, rb, nb, kb, a, b, as, bs);
-                    uint8_t *sa = smem + sl * SL_BYTES, *sb = sa + 4 * A_BYTES;
-                    for (int q = 0; q < 4; ++q) bulk_g2s(smem_u32(sa + q * A_BYTES), a + q * as, A_BYTES, fb);
-                    for (int q = 0; q < 4; ++q) bulk_g2s(smem_u32(sb + q * B_BYTES), b + q * bs, B_BYTES, fb);
-                    if (++sl == 4) { sl = 0; phl ^= 1; }
-                }
-            }
-        }
-    } else if (warp == 1) {
-        if (lane == 0) {
-            int sh = 0, sl = 0;
-            uint32_t phh = 0, phl = 0;
-            int64_t tile_i = 0;
-            for (int64_t it = blockIdx.x; it < n_items; it += gridDim.x, ++tile_i) {
-                int party, kb0, kb1, rb, nb;
-                decode(it, party, kb0, kb1, rb, nb);
-                if (tile_i > 0) {   // previous tile's pass-L accumulators read out
-                    mbar_wait(smem_u32(tfree), (uint32_t)((tile_i - 1) & 1));
-                    tc_fence_after();
-                }
-                for (int kb = kb0; kb < kb1; ++kb) {
-                    mbar_wait(smem_u32(&fullH[sh]), phh);
-                    tc_fence_after();
-                    const uint32_t sa = smem_u32(smem + sh * SH_BYTES), sb = sa + L * A_BYTES;
-#pragma unroll
-                    for (int p = 0; p < 8; ++p) {
-                        const uint64_t ad = smem_desc(sa + p * A_BYTES, 128, 256);
-#pragma unroll
-                        for (int q = (p < 4 ? 4 - p : 0); q < 8 - p; ++q)
-                            tc_mma_i8(tmem + (uint32_t)((p + q - 4) * BN), ad, smem_desc(sb + q * B_BYTES, 128, 256),
-                                      IDESC, (kb > kb0 || p > 0) ? 1u : 0u);
-                    }
-                    tc_commit(smem_u32(&emptyH[sh]));
-                    if (++sh == 2) { sh = 0; phh ^= 1; }
-                }
-                tc_commit(smem_u32(accf));
-                mbar_wait(smem_u32(acce), (uint32_t)(tile_i & 1));
-                tc_fence_after();
-                for (int kb = kb0; kb < kb1; ++kb) {
-                    mbar_wait(smem_u32(&fullL[sl]), phl);
-                    tc_fence_after();
-                    const uint32_t sa = smem_u32(smem + sl * SL_BYTES), sb = sa + 4 * A_BYTES;
-#pragma unroll
-                    for (int p = 0; p < 4; ++p) {
-                        const uint64_t ad = smem_desc(sa + p * A_BYTES, 128, 256);
-#pragma unroll
-                        for (int q = 0; q < 4 - p; ++q)
-                            tc_mma_i8(tmem + (uint32_t)((p + q) * BN), ad, smem_desc(sb + q * B_BYTES, 128, 256),
-                                      IDESC, (kb > kb0 || p > 0) ? 1u : 0u);
-                    }
-                    tc_commit(smem_u32(&emptyL[sl]));
-                    if (++sl == 4) { sl = 0; phl ^= 1; }
-                }
-                tc_commit(smem_u32(accf));
-            }
-        }
-    } else {
-        const int quarter = warp & 3;
-        const int rl = quarter * 32 + lane;
-        const uint32_t lane_base = tmem + ((uint32_t)(quarter * 32) << 16);
-        int64_t tile_i = 0;
-        for (int64_t it = blockIdx.x; it < n_items; it += gridDim.x, ++tile_i) {
-            int party, kb0, kb1, rb, nb;
-            decode(it, party, kb0, kb1, rb, nb);
-            const int64_t row = (int64_t)rb * BM + rl;
-            const int64_t col0 = (int64_t)nb * BN;
-            mbar_wait(smem_u32(accf), 0);   // pass H of this tile (2 completions per tile)
-            tc_fence_after();
-#pragma unroll 1
-            for (int j0 = 0; j0 < BN; j0 += 16) {
-                uint32_t hi[16];
-#pragma unroll
-                for (int j = 0; j < 16; ++j) hi[j] = 0;
-#pragma unroll
-                for (int s = 0; s < 4; ++s) {
-                    uint32_t r[16];
-                    tmem_ld16(lane_base + (uint32_t)(s * BN + j0), r);
-#pragma unroll
-                    for (int j = 0; j < 16; ++j) hi[j] += r[j] << (8 * s);
-                }
-#pragma unroll
-                for (int j = 0; j < 16; ++j) hi_buf[(j0 + j) * BM + rl] = hi[j];
-            }
-            tc_fence_before();
-            mbar_arrive(smem_u32(acce));
-            mbar_wait(smem_u32(accf), 1);   // pass L of this tile
-            tc_fence_after();
-            // pass-L chunks: low + high 2^32; TMEM is released after the last chunk's loads so the
-            // stores of this tile overlap the next tile's pass-H MMAs
-#pragma unroll 1
-            for (int j0 = 0; j0 < BN; j0 += 16) {
-                T acc[16];
-#pragma unroll
-                for (int j = 0; j < 16; ++j) acc[j] = (T)hi_buf[(j0 + j) * BM + rl] << 32;
-#pragma unroll
-                for (int s = 0; s < 4; ++s) {
-                    uint32_t r[16];
-                    tmem_ld16(lane_base + (uint32_t)(s * BN + j0), r);
-#pragma unroll
-                    for (int j = 0; j < 16; ++j) acc[j] += (T)r[j] << (8 * s);
-                }
-                if (j0 == BN - 16) {   // TMEM read out: the next tile's pass H may start
-                    tc_fence_before();
-                    mbar_arrive(smem_u32(tfree));
-                }
-                if (row < P.M && !(P.debug & 1)) {
-#pragma unroll
-                    for (int j = 0; j < 16; ++j) {
-                        const int64_t col = col0 + j0 + j;
-                        if (col >= P.N) break;
-                        const int64_t o = row * P.N + col;
-                        switch (P.mode) {
-                        case 0: P.C[party][o] = acc[j]; break;
-                        case 1: P.C[party][o] = trunc_share<T>(acc[j] + P.Z[party][o], party, P.trunc); break;
-                        case 2: P.C[0][o] = acc[j] - P.Z[0][o]; break;
-                        default: atomicAdd((unsigned long long *)(P.partial + (int64_t)(party - P.party_base) * P.M * P.N + o), acc[j]);
-                        }
-                    }
-                }
-            }
-        }
-    }
-    tc_fence_before();
-    __syncthreads();
-    if (warp == 2) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tmem));
-}
-
-template <int STAGES>
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(192, 1) tc_ring_gemm64_2sm(const TcParams<uint64_t> P) {
-    using T = uint64_t;
-    constexpr int BN = 128, HB = 64, L = 8;
-    extern __shared__ __align__(1024) uint8_t smem[];
-    constexpr int A_BYTES = BM * BK, HB_BYTES = HB * BK;          // own A tile, own half of B
-    constexpr int STAGE_BYTES = L * (A_BYTES + HB_BYTES);
-    constexpr uint32_t IDESC = idesc_i8(2 * BM, BN);
-    uint64_t *full = (uint64_t *)(smem + STAGES * STAGE_BYTES);
-    uint64_t *empty = full + STAGES;
-    uint64_t *accf = empty + STAGES;
-    uint64_t *acce = accf + 1;
-    uint32_t *tmem_slot = (uint32_t *)(acce + 1);
-
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const uint32_t rank = cluster_rank();
-    const int party = P.party_base + blockIdx.z % P.nparty, split = blockIdx.z / P.nparty;
-    const int nb = blockIdx.x >> 1;
-    const int rb = blockIdx.y * 2 + (int)rank;                      // this CTA's 128-row A tile
-    const int nkb = P.nkb_lo + P.nkb_hi;
-    const int kb0 = split * P.kb_per_split;
-    const int kb1 = min(kb0 + P.kb_per_split, nkb);
-
-    if (threadIdx.x == 0) {
-        for (int s = 0; s < STAGES; ++s) {
-            mbar_init(smem_u32(&full[s]), rank == 0 ? 2 : 1);   // leader: own tx + peer's forward
-            mbar_init(smem_u32(&empty[s]), 1);
-        }
-        mbar_init(smem_u32(accf), 1);
-        mbar_init(smem_u32(acce), 8);                            // 4 local + 4 peer epilogue warps
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    if (warp == 2) {
-        asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_u32(tmem_slot)));
-        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
-    }
-    tc_fence_before();
-    cluster_sync_all();
-    tc_fence_after();
-    const uint32_t tmem = *tmem_slot;
-
-    if (warp == 0) {
-        if (lane == 0) {
-            // ---------------- TMA producer (both CTAs): own A tile + own half of B ----------------
-            int stage = 0;
-            uint32_t phase = 0;
-            for (int pass = 0; pass < 2; ++pass) {
-                const int nl = pass == 0 ? 4 : 8;
-                for (int kb = kb0; kb < kb1; ++kb) {
-                    mbar_wait(smem_u32(&empty[stage]), phase ^ 1);
-                    const uint32_t fb = smem_u32(&full[stage]);
-                    mbar_expect_tx(fb, (uint32_t)(nl * (A_BYTES + HB_BYTES)));
-                    const bool lo = kb < P.nkb_lo;
-                    const int kk = lo ? kb : kb - P.nkb_lo;
-                    const int nk = lo ? P.nkb_lo : P.nkb_hi;
-                    const uint8_t *a = (lo ? P.A_lo[party] : P.A_hi[party]) + ((int64_t)rb * nk + kk) * A_BYTES;
-                    const uint8_t *b = (lo ? P.B_lo[party] : P.B_hi[party]) + ((int64_t)nb * nk + kk) * (BN * BK) +
-                                       rank * HB_BYTES;
-                    const int64_t as = lo ? P.a_stride_lo : P.a_stride_hi, bs = lo ? P.b_stride_lo : P.b_stride_hi;
-                    uint8_t *sa = smem + stage * STAGE_BYTES, *sb = sa + L * A_BYTES;
-                    for (int p = 0; p < nl; ++p) bulk_g2s(smem_u32(sa + p * A_BYTES), a + p * as, A_BYTES, fb);
-                    for (int q = 0; q < nl; ++q) bulk_g2s(smem_u32(sb + q * HB_BYTES), b + q * bs, HB_BYTES, fb);
-                    if (++stage == STAGES) { stage = 0; phase ^= 1; }
-                }
-            }
-        }
-    } else if (warp == 1) {
-        if (lane == 0 && rank == 0) {
-            // ---------------- MMA issuer (leader only) ----------------
-            int stage = 0;
-            uint32_t phase = 0;
-            for (int pass = 0; pass < 2; ++pass) {
-                if (pass == 1) {
-                    mbar_wait(smem_u32(acce), 0);   // both CTAs drained pass L
-                    tc_fence_after();
-                }
-                for (int kb = kb0; kb < kb1; ++kb) {
-                    mbar_wait(smem_u32(&full[stage]), phase);   // own bytes landed + peer forwarded
-                    tc_fence_after();
-                    const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES), sb = sa + L * A_BYTES;
-                    if (pass == 0) {
-#pragma unroll
-                        for (int p = 0; p < 4; ++p) {
-                            const uint64_t ad = smem_desc(sa + p * A_BYTES, 128, 256);
-#pragma unroll
-                            for (int q = 0; q < 4 - p; ++q)
-                                tc_mma_i8_2sm(tmem + (uint32_t)((p + q) * BN), ad, smem_desc(sb + q * HB_BYTES, 128, 256),
-                                              IDESC, (kb > kb0 || p > 0) ? 1u : 0u);
-                        }
-                    } else {
-#pragma unroll
-                        for (int p = 0; p < 8; ++p) {
-                            const uint64_t ad = smem_desc(sa + p * A_BYTES, 128, 256);
-#pragma unroll
-                            for (int q = (p < 4 ? 4 - p : 0); q < 8 - p; ++q)
-                                tc_mma_i8_2sm(tmem + (uint32_t)((p + q - 4) * BN), ad,
-                                              smem_desc(sb + q * HB_BYTES, 128, 256), IDESC, (kb > kb0 || p > 0) ? 1u : 0u);
-                        }
-                    }
-                    tc_commit_2sm(smem_u32(&empty[stage]));   // frees the stage in BOTH CTAs
-                    if (++stage == STAGES) { stage = 0; phase ^= 1; }
-                }
-                tc_commit_2sm(smem_u32(accf));
-            }
-        } else if (lane == 0 && rank == 1) {
-            // ---------------- peer: forward "stage landed" to the leader's full barrier ----------------
-            int stage = 0;
-            uint32_t phase = 0;
-            const uint32_t leader_full0 = map_to_rank(smem_u32(&full[0]), 0);
-            for (int pass = 0; pass < 2; ++pass)
-                for (int kb = kb0; kb < kb1; ++kb) {
-                    mbar_wait(smem_u32(&full[stage]), phase);
-                    mbar_arrive_remote(leader_full0 + stage * 8);
-                    if (++stage == STAGES) { stage = 0; phase ^= 1; }
-                }
-        }
-    } else {
-        // ---------------- epilogue warps 2..5 (both CTAs, own 128 rows) ----------------
-        const int quarter = warp & 3;
-        const int64_t row = (int64_t)rb * BM + quarter * 32 + lane;
-        const uint32_t lane_base = tmem + ((uint32_t)(quarter * 32) << 16);
-        const int64_t col0 = (int64_t)nb * BN;
-        const uint32_t leader_acce = map_to_rank(smem_u32(acce), 0);
-        mbar_wait(smem_u32(accf), 0);
-        tc_fence_after();
-#pragma unroll 1
-        for (int j0 = 0; j0 < BN; j0 += 16) {
-            T acc[16];
-#pragma unroll
-            for (int j = 0; j < 16; ++j) acc[j] = 0;
-#pragma unroll
-            for (int s = 0; s < 4; ++s) {
-                uint32_t r[16];
-                tmem_ld16(lane_base + (uint32_t)(s * BN + j0), r);
-#pragma unroll
-                for (int j = 0; j < 16; ++j) acc[j] += (T)r[j] << (8 * s);
-            }
-            if (j0 == BN - 16) {   // this warp's TMEM lanes fully read: tell the leader
-                tc_fence_before();
-                __syncwarp();
-                if (lane == 0) mbar_arrive_remote(leader_acce);
-            }
-            if (row < P.M) {
-#pragma unroll
-                for (int j = 0; j < 16; ++j) {
-                    const int64_t col = col0 + j0 + j;
-                    if (col >= P.N) break;
-                    const int64_t o = row * P.N + col;
-                    if (P.mode == 3) atomicAdd((unsigned long long *)(P.partial + (int64_t)(party - P.party_base) * P.M * P.N + o), acc[j]);
-                    else P.C[P.mode == 2 ? 0 : party][o] = acc[j];
-                }
-            }
-        }
-        mbar_wait(smem_u32(accf), 1);
-        tc_fence_after();
-#pragma unroll 1
-        for (int j0 = 0; j0 < BN; j0 += 16) {
-            uint32_t hi[16];
-#pragma unroll
-            for (int j = 0; j < 16; ++j) hi[j] = 0;
-#pragma unroll
-            for (int s = 0; s < 4; ++s) {
-                uint32_t r[16];
-                tmem_ld16(lane_base + (uint32_t)(s * BN + j0), r);
-#pragma unroll
-                for (int j = 0; j < 16; ++j) hi[j] += r[j] << (8 * s);
-            }
-            if (row < P.M) {
-#pragma unroll
-                for (int j = 0; j < 16; ++j) {
-                    const int64_t col = col0 + j0 + j;
-                    if (col >= P.N) break;
-                    const int64_t o = row * P.N + col;
-                    const T h = (T)hi[j] << 32;
-                    switch (P.mode) {
-                    case 0: P.C[party][o] = P.C[party][o] + h; break;
-                    case 1: P.C[party][o] = trunc_share<T>(P.C[party][o] + h + P.Z[party][o], party, P.trunc); break;
-                    case 2: P.C[0][o] = P.C[0][o] + h - P.Z[0][o]; break;
-                    default: atomicAdd((unsigned long long *)(P.partial + (int64_t)(party - P.party_base) * P.M * P.N + o), h);
-                    }
-                }
-            }
-        }
-    }
-    tc_fence_before();
-    cluster_sync_all();
-    if (warp == 2) asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, 512;" ::"r"(tmem));
-}
-
 template <typename T>
 __global__ void tc_finalize_kernel(const TcParams<T> P, int mode) {
     const int64_t total = P.M * P.N * P.nparty;
@@ -1208,7 +560,6 @@ template <int l>
 constexpr size_t smem_bytes() {
     return (size_t)Cfg<l>::STAGES * Cfg<l>::L * (BM * BK + Cfg<l>::BN * BK) + 256;
 }
-constexpr size_t smem_pair_bytes() { return (size_t)4 * 8 * (BM * BK + 64 * BK) + 256; }
 
 static inline int64_t rup(int64_t x, int64_t m) { return (x + m - 1) / m * m; }
 
@@ -1267,35 +618,7 @@ static psml_status launch_gemm(TcParams<typename Cfg<l>::T> P, int64_t Mp, int64
     {
         ProfScope prof(PROF_TC, s, (double)P.M * P.N * (double)(P.nkb_lo + P.nkb_hi) * BK * P.nparty);
         if constexpr (l == 64) {
-            static const bool pair = getenv("PSML_TC_2SM") && getenv("PSML_TC_2SM")[0] == '1';
-            if (pair) {   // CTA-pair variant (cta_group::2); bit-exact, not faster yet
-                auto kern = tc_ring_gemm64_2sm<4>;
-                static bool attr_set = false;
-                if (!attr_set) {
-                    PSML_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_pair_bytes()));
-                    attr_set = true;
-                }
-                dim3 g2((unsigned)(2 * (Np / BN)), (unsigned)(Mp / (2 * BM)), grid.z);   // x = (n tile, pair rank)
-                kern<<<g2, 192, smem_pair_bytes(), s>>>(P);
-            } else if (getenv("PSML_TC_V2")) {   // previous schedule (pass-L partial via HBM)
-                auto kern = tc_ring_gemm64_v2<Cfg<l>::STAGES>;
-                static bool attr_set = false;
-                if (!attr_set) {
-                    PSML_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_bytes<l>()));
-                    attr_set = true;
-                }
-                kern<<<grid, 192, smem_bytes<l>(), s>>>(P);
-            } else if (getenv("PSML_TC_V5")) {   // persistent v5: bit-exact, not faster than v4 yet
-                auto kern = tc_ring_gemm64_v5;
-                static bool attr_set = false;
-                if (!attr_set) {
-                    PSML_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_v4_bytes()));
-                    attr_set = true;
-                }
-                const int64_t items = (int64_t)grid.x * grid.y * grid.z;
-                const int ctas = (int)std::min<int64_t>(items, sm_count);
-                kern<<<ctas, 192, smem_v4_bytes(), s>>>(P, (int)grid.x, (int)grid.y, splits);
-            } else {
+            {
                 auto kern = tc_ring_gemm64_v4;
                 static bool attr_set = false;
                 if (!attr_set) {

@@ -12,7 +12,9 @@ import sys
 
 CLASSES = [("seg_gemm_kernel", "ring_gemm_cuda_core"), ("tc_seg_kernel", "ring_gemm_tcgen05"),
            ("msb_chain_pair_kernel", "msb_relu_eq9_rounds"), ("had_fused_kernel", "hadamard_rounds"),
-           ("deal_prg_kernel", "dealer"), ("ring_gemm_cl_grouped", "dealer"), ("open_list_kernel", "beaver_mask")]
+           ("deal_prg_kernel", "dealer"), ("ring_gemm_cl_grouped", "dealer"), ("open_list_kernel", "beaver_mask"),
+           ("tc_ring_gemm64_v4", "ring_gemm_tc_l64"), ("tc_ring_gemm_kernel", "ring_gemm_tc_l32"),
+           ("split_kernel", "ring_gemm_limb_split")]
 SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "KB": 1e3, "MB": 1e6, "GB": 1e9}
 
 rep, out = sys.argv[1], sys.argv[2]
