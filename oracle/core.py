@@ -40,6 +40,15 @@ def lib():
         L.or_delta_csr_encode.restype = c_i64
         L.or_delta_csr_apply.argtypes = [c_i, c_i64, c_i64, ctypes.c_int32, vp, vp, vp, vp, vp]
         L.or_num_threads.restype = c_i
+        L.or_dcf_key_words.argtypes = [c_i]
+        L.or_dcf_key_words.restype = c_i64
+        L.or_dcf_gen.argtypes = [c_i, c_i, c_u64, c_u64, c_u64, c_u64, c_u64, c_u64, vp, vp]
+        L.or_dcf_eval.argtypes = [c_i, c_i, c_i, vp, c_u64]
+        L.or_dcf_eval.restype = c_u64
+        L.or_fss_words.argtypes = [c_i]
+        L.or_fss_words.restype = c_i64
+        L.or_fss_dealer.argtypes = [c_i, c_u64, c_u64, c_i64, vp, vp]
+        L.or_fss_drelu.argtypes = [c_i, vp, vp, c_i64, vp, vp, vp, vp, vp]
     return _lib
 
 
@@ -228,6 +237,48 @@ def secure_eq9(z, mat, htrip, l=64, f=13):
     y0 = ((r0[:n] - r0[n:]) & m).reshape(shape)
     y1 = ((r1[:n] - r1[n:]) & m).reshape(shape)
     return y0, y1
+
+
+# ---------------------------------------------------------------------------------------------
+# one-round secure comparison by FSS (DCF, R22)
+# ---------------------------------------------------------------------------------------------
+def dcf_gen(l, n_bits, alpha, beta, seed0, seed1):
+    """DCF keys of f(x) = beta * [x < alpha] on n_bits inputs; seeds are (lo, hi) 128-bit pairs."""
+    kw = lib().or_dcf_key_words(n_bits)
+    k0, k1 = np.empty(kw, np.uint64), np.empty(kw, np.uint64)
+    lib().or_dcf_gen(l, n_bits, alpha, beta, seed0[0], seed0[1], seed1[0], seed1[1], _p(k0), _p(k1))
+    return k0, k1
+
+
+def dcf_eval(l, n_bits, b, key, x):
+    return lib().or_dcf_eval(l, n_bits, b, _p(_u64(key)), int(x))
+
+
+def fss_dealer(seed, call_id, n, l=64):
+    w = lib().or_fss_words(l) * n
+    m0, m1 = np.empty(w, np.uint64), np.empty(w, np.uint64)
+    lib().or_fss_dealer(l, seed, call_id, n, _p(m0), _p(m1))
+    return m0, m1
+
+
+def fss_drelu(x, mat, l=64, trace=False):
+    """Arithmetic shares of DReLU(x) = [x >= 0] after ONE opening (xhat = x + r) + DCF evaluation."""
+    x0, x1 = _u64(x[0]).reshape(-1), _u64(x[1]).reshape(-1)
+    n = x0.size
+    d0, d1, xh = np.empty(n, np.uint64), np.empty(n, np.uint64), np.empty(n, np.uint64)
+    lib().or_fss_drelu(l, _p(x0), _p(x1), n, _p(mat[0]), _p(mat[1]), _p(d0), _p(d1), _p(xh))
+    shape = np.shape(x[0])
+    out = (d0.reshape(shape), d1.reshape(shape))
+    return (out, xh.reshape(shape)) if trace else out
+
+
+def secure_relu_fss(x, mat, htrip, l=64):
+    """ReLU(x) = x (.) DReLU(x): the FSS comparison round, then one Beaver Hadamard round."""
+    d = fss_drelu(x, mat, l)
+    r = beaver_hadamard((_u64(x[0]).reshape(-1), _u64(x[1]).reshape(-1)),
+                        (d[0].reshape(-1), d[1].reshape(-1)), htrip, l)
+    shape = np.shape(x[0])
+    return (r[0].reshape(shape), r[1].reshape(shape)), d
 
 
 # ---------------------------------------------------------------------------------------------

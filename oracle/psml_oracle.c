@@ -421,6 +421,190 @@ EXPORT void or_delta_csr_apply(int l, int64_t rows, int64_t cols, int32_t is_csr
     }
 }
 
+/* ------------------------------------------------------------------------------------------ */
+/* One-round secure comparison by function secret sharing (R22).      */
+/* Distributed comparison function (DCF) of Boyle, Chandran, Gilboa, Gupta, Ishai, Kumar and    */
+/* Rathee, "Function Secret Sharing for Mixed-Mode and Fixed-Point Secure Computation"          */
+/* (EUROCRYPT 2021), Fig. 1: f_{alpha,beta}(x) = beta if x < alpha else 0 over n-bit inputs      */
+/* (bits taken most significant first), output group Z_{2^l}, seeds of lambda = 128 bits.       */
+/* The paper only says Eq. 9 is computed "in GPUs"; this is the one-round       */
+/* alternative to the Kogge-Stone A2B of R9.                                                    */
+/* ------------------------------------------------------------------------------------------ */
+typedef struct { uint64_t lo, hi; } seed128;
+
+/* G: {0,1}^128 -> (s^L, v^L, t^L, s^R, v^R, t^R): one ChaCha20 block keyed by the seed (16 bytes
+ * little endian || 16 zero bytes), counter 0, nonce = tag "DCFG" || 8 zero bytes.  Words 0-3 s^L,
+ * 4-7 s^R, 8-9 v^L, 10-11 v^R (little endian u64, reduced mod 2^l), bit 0 of word 12 t^L, of 13 t^R. */
+static void dcf_G(int l, seed128 s, seed128 *sL, uint64_t *vL, int *tL, seed128 *sR, uint64_t *vR, int *tR) {
+    uint32_t key[8] = {(uint32_t)s.lo, (uint32_t)(s.lo >> 32), (uint32_t)s.hi, (uint32_t)(s.hi >> 32), 0, 0, 0, 0};
+    uint32_t nonce[3] = {0x47464344u /* "DCFG" */, 0, 0};
+    uint32_t w[16];
+    or_chacha20_block(key, 0, nonce, w);
+    uint64_t m = ring_mask(l);
+    sL->lo = (uint64_t)w[0] | ((uint64_t)w[1] << 32);
+    sL->hi = (uint64_t)w[2] | ((uint64_t)w[3] << 32);
+    sR->lo = (uint64_t)w[4] | ((uint64_t)w[5] << 32);
+    sR->hi = (uint64_t)w[6] | ((uint64_t)w[7] << 32);
+    *vL = ((uint64_t)w[8] | ((uint64_t)w[9] << 32)) & m;
+    *vR = ((uint64_t)w[10] | ((uint64_t)w[11] << 32)) & m;
+    *tL = (int)(w[12] & 1);
+    *tR = (int)(w[13] & 1);
+}
+
+static uint64_t convert(int l, seed128 s) { return s.lo & ring_mask(l); }   /* Convert_G: low word */
+static inline uint64_t neg_if(int t, uint64_t v, uint64_t m) { return (t ? (0 - v) : v) & m; }
+
+/* DCF key words (per party): [0] seed.lo, [1] seed.hi, then per level i = 1..n: s_CW.lo, s_CW.hi,
+ * V_CW, t_CW^L | t_CW^R << 1; then CW^(n+1).  4n + 3 words. */
+EXPORT int64_t or_dcf_key_words(int n_bits) { return 4 * (int64_t)n_bits + 3; }
+
+/* Gen(1^lambda, alpha, beta) of Fig. 1 with the two root seeds given (drawn by the caller's PRG). */
+EXPORT void or_dcf_gen(int l, int n_bits, uint64_t alpha, uint64_t beta, uint64_t s0lo, uint64_t s0hi,
+                       uint64_t s1lo, uint64_t s1hi, uint64_t *k0, uint64_t *k1) {
+    uint64_t m = ring_mask(l);
+    seed128 s[2] = {{s0lo, s0hi}, {s1lo, s1hi}};
+    int t[2] = {0, 1};
+    uint64_t Va = 0;
+    k0[0] = s0lo; k0[1] = s0hi; k1[0] = s1lo; k1[1] = s1hi;
+    for (int i = 1; i <= n_bits; ++i) {
+        seed128 sL[2], sR[2];
+        uint64_t vL[2], vR[2];
+        int tL[2], tR[2];
+        for (int b = 0; b < 2; ++b) dcf_G(l, s[b], &sL[b], &vL[b], &tL[b], &sR[b], &vR[b], &tR[b]);
+        int ai = (int)((alpha >> (n_bits - i)) & 1);               /* alpha_i, MSB first */
+        /* Keep = the child on alpha's path, Lose = the other one */
+        seed128 *sKeep = ai ? sR : sL, *sLose = ai ? sL : sR;
+        uint64_t *vKeep = ai ? vR : vL, *vLose = ai ? vL : vR;
+        int *tKeep = ai ? tR : tL;
+        seed128 scw = {sLose[0].lo ^ sLose[1].lo, sLose[0].hi ^ sLose[1].hi};
+        uint64_t Vcw = neg_if(t[1], (vLose[1] - vLose[0] - Va) & m, m);
+        if (ai == 1) Vcw = (Vcw + neg_if(t[1], beta, m)) & m;      /* Lose = L: x < alpha below here */
+        Va = (Va - vKeep[1] + vKeep[0] + neg_if(t[1], Vcw, m)) & m;
+        int tcwL = tL[0] ^ tL[1] ^ ai ^ 1, tcwR = tR[0] ^ tR[1] ^ ai;
+        int tcwKeep = ai ? tcwR : tcwL;
+        int64_t o = 2 + 4 * (int64_t)(i - 1);
+        k0[o] = k1[o] = scw.lo;
+        k0[o + 1] = k1[o + 1] = scw.hi;
+        k0[o + 2] = k1[o + 2] = Vcw;
+        k0[o + 3] = k1[o + 3] = (uint64_t)(tcwL | (tcwR << 1));
+        for (int b = 0; b < 2; ++b) {
+            seed128 ns = sKeep[b];
+            if (t[b]) { ns.lo ^= scw.lo; ns.hi ^= scw.hi; }
+            int nt = tKeep[b] ^ (t[b] & tcwKeep);
+            s[b] = ns;
+            t[b] = nt;
+        }
+    }
+    uint64_t last = neg_if(t[1], (convert(l, s[1]) - convert(l, s[0]) - Va) & m, m);
+    k0[2 + 4 * (int64_t)n_bits] = k1[2 + 4 * (int64_t)n_bits] = last;
+}
+
+/* Eval(b, k_b, x) of Fig. 1: party b's additive share of f_{alpha,beta}(x). */
+EXPORT uint64_t or_dcf_eval(int l, int n_bits, int b, const uint64_t *k, uint64_t x) {
+    uint64_t m = ring_mask(l);
+    seed128 s = {k[0], k[1]};
+    int t = b;
+    uint64_t V = 0;
+    for (int i = 1; i <= n_bits; ++i) {
+        int64_t o = 2 + 4 * (int64_t)(i - 1);
+        seed128 scw = {k[o], k[o + 1]};
+        uint64_t Vcw = k[o + 2];
+        int tcwL = (int)(k[o + 3] & 1), tcwR = (int)((k[o + 3] >> 1) & 1);
+        seed128 sL, sR;
+        uint64_t vL, vR;
+        int tL, tR;
+        dcf_G(l, s, &sL, &vL, &tL, &sR, &vR, &tR);
+        if (t) {
+            sL.lo ^= scw.lo; sL.hi ^= scw.hi; tL ^= tcwL;
+            sR.lo ^= scw.lo; sR.hi ^= scw.hi; tR ^= tcwR;
+        }
+        int xi = (int)((x >> (n_bits - i)) & 1);
+        if (!xi) {
+            V = (V + neg_if(b, (vL + (t ? Vcw : 0)) & m, m)) & m;
+            s = sL; t = tL;
+        } else {
+            V = (V + neg_if(b, (vR + (t ? Vcw : 0)) & m, m)) & m;
+            s = sR; t = tR;
+        }
+    }
+    uint64_t last = k[2 + 4 * (int64_t)n_bits];
+    V = (V + neg_if(b, (convert(l, s) + (t ? last : 0)) & m, m)) & m;
+    return V;
+}
+
+/*
+ * FSS DReLU material (R22), per element e and party b, as fss_words(l) = 4(l-1) + 5
+ * words in structure-of-arrays order (word w of element e at mat_b[w * n + e]):
+ *   w = 0: r_b        additive share of the input mask r = PRG(seed, "FR", id)[e]
+ *                     (r_0 = PRG("F0"), r_1 = r - r_0)
+ *   w = 1: sA_b       additive share of s = MSB(r)  (sA_0 = PRG("FS"), sA_1 = s - sA_0)
+ *   w = 2..:          DCF key of f_{alpha,beta} with n = l - 1 input bits, alpha = r mod 2^(l-1),
+ *                     beta = 1 - 2s (mod 2^l); root seeds (PRG("K0")[2e], [2e+1]) and
+ *                     (PRG("K1")[2e], [2e+1]).
+ */
+EXPORT int64_t or_fss_words(int l) { return 4 * (int64_t)(l - 1) + 5; }
+
+EXPORT void or_fss_dealer(int l, uint64_t seed, uint64_t call_id, int64_t n, uint64_t *mat0, uint64_t *mat1) {
+    uint64_t m = ring_mask(l);
+    int nb = l - 1;
+    int64_t kw = or_dcf_key_words(nb);
+    uint64_t *r = malloc(sizeof(uint64_t) * n), *r0 = malloc(sizeof(uint64_t) * n), *sa0 = malloc(sizeof(uint64_t) * n);
+    uint64_t *K0 = malloc(sizeof(uint64_t) * 2 * n), *K1 = malloc(sizeof(uint64_t) * 2 * n);
+    or_prg(l, seed, 0x00005246u /* "FR" */, call_id, 0, n, r);
+    or_prg(l, seed, 0x00003046u /* "F0" */, call_id, 0, n, r0);
+    or_prg(l, seed, 0x00005346u /* "FS" */, call_id, 0, n, sa0);
+    or_prg(64, seed, 0x0000304Bu /* "K0" */, call_id, 0, 2 * n, K0);
+    or_prg(64, seed, 0x0000314Bu /* "K1" */, call_id, 0, 2 * n, K1);
+#pragma omp parallel for schedule(static)
+    for (int64_t e = 0; e < n; ++e) {
+        uint64_t k0[4 * 64 + 3], k1[4 * 64 + 3];
+        uint64_t sbit = (r[e] >> (l - 1)) & 1;
+        uint64_t alpha = r[e] & (((uint64_t)1 << nb) - 1);
+        uint64_t beta = (1 - 2 * sbit) & m;
+        or_dcf_gen(l, nb, alpha, beta, K0[2 * e], K0[2 * e + 1], K1[2 * e], K1[2 * e + 1], k0, k1);
+        mat0[e] = r0[e];
+        mat1[e] = (r[e] - r0[e]) & m;
+        mat0[n + e] = sa0[e];
+        mat1[n + e] = (sbit - sa0[e]) & m;
+        for (int64_t w = 0; w < kw; ++w) {
+            mat0[(2 + w) * n + e] = k0[w];
+            mat1[(2 + w) * n + e] = k1[w];
+        }
+    }
+    free(r); free(r0); free(sa0); free(K0); free(K1);
+}
+
+/*
+ * FSS DReLU, both parties (R22).  Round 1 (the only opening): xhat = (x_0 + r_0) +
+ * (x_1 + r_1) = x + r.  Then locally, with c = MSB(xhat) and xhat' = xhat mod 2^(l-1):
+ *   MSB(x) = c XOR s XOR [xhat' < r']   (x = xhat - r: a borrow out of the low l-1 bits flips the MSB)
+ *   [s XOR borrow]_b = sA_b + Eval(b, k_b, xhat')            (the DCF pays beta = 1 - 2s)
+ *   [MSB]_b = c ? [b = 0] - [s XOR borrow]_b : [s XOR borrow]_b ;  DReLU_b = [b = 0] - [MSB]_b.
+ * Outputs arithmetic shares of DReLU(x) = 1{x >= 0} (signed), and the opened xhat (trace).
+ */
+EXPORT void or_fss_drelu(int l, const uint64_t *x0, const uint64_t *x1, int64_t n, const uint64_t *mat0,
+                         const uint64_t *mat1, uint64_t *d0, uint64_t *d1, uint64_t *xhat_out) {
+    uint64_t m = ring_mask(l);
+    int nb = l - 1;
+    int64_t kw = or_dcf_key_words(nb);
+    const uint64_t *mat[2] = {mat0, mat1};
+    uint64_t *d[2] = {d0, d1};
+#pragma omp parallel for schedule(static)
+    for (int64_t e = 0; e < n; ++e) {
+        uint64_t xhat = ((x0[e] + mat0[e]) + (x1[e] + mat1[e])) & m;   /* Eq. 4-5 style opening */
+        if (xhat_out) xhat_out[e] = xhat;
+        uint64_t c = (xhat >> (l - 1)) & 1;
+        uint64_t xlow = xhat & (((uint64_t)1 << nb) - 1);
+        uint64_t k[4 * 64 + 3];
+        for (int b = 0; b < 2; ++b) {
+            for (int64_t w = 0; w < kw; ++w) k[w] = mat[b][(2 + w) * n + e];
+            uint64_t sb = (mat[b][n + e] + or_dcf_eval(l, nb, b, k, xlow)) & m;
+            uint64_t msb = c ? (((uint64_t)(b == 0)) - sb) & m : sb;
+            d[b][e] = (((uint64_t)(b == 0)) - msb) & m;
+        }
+    }
+}
+
 EXPORT int or_num_threads(void) {
 #ifdef _OPENMP
     extern int omp_get_max_threads(void);
