@@ -226,6 +226,33 @@ psml_status psml_secure_eq9(psml_ctx ctx, const void *const x[2], int64_t n,
                             const void *const V[2], const void *const Z[2], void *const y[2],
                             psml_stream stream);
 
+/* One-round secure comparison by function secret sharing (R22): the
+ * distributed comparison function of Boyle et al. (EUROCRYPT 2021, Fig. 1) replaces the
+ * 1 + log2(l)-round Kogge-Stone A2B of psml_secure_msb for DReLU.  Z_2^64 only
+ * (PSML_ERR_UNSUPPORTED otherwise).  psml_fss_dealer writes, per element and party, 257 words in
+ * structure-of-arrays order (word w of element e at mat[i][w * n + e]): the input-mask share r_i,
+ * the share of s = MSB(r), the party's 128-bit DCF root seed and the 63 levels of correction words
+ * + the final one (layout in fss.cuh; streams keyed by (seed, "FR"/"F0"/"FS"/"K0"/"K1", call_id)).
+ * psml_fss_material_words(ring, n) = 257 n for l = 64, -1 otherwise.
+ * psml_secure_drelu_fss: ONE opening (xhat = x + r), then each party evaluates its DCF key on the
+ * low 63 bits of xhat: arithmetic shares of DReLU(x) = [x >= 0 signed] in drelu[2];
+ * xhat_trace (nullable, device, n words) receives the opened value.  psml_secure_relu_fss adds
+ * the Beaver Hadamard y = x . DReLU(x) (triplet U, V, Z of n elements), drelu nullable.
+ * Split deployment: psml_fss_mask writes party i's message x_i + r_i; after the exchange
+ * psml_fss_open_drelu opens xhat = msg_send + msg_recv and writes party i's DReLU share. */
+int64_t psml_fss_material_words(psml_ring ring, int64_t n);
+psml_status psml_fss_dealer(psml_ring ring, uint64_t seed, uint64_t call_id, int64_t n, void *const mat[2],
+                            psml_stream stream);
+psml_status psml_secure_drelu_fss(psml_ctx ctx, const void *const x[2], int64_t n, const void *const mat[2],
+                                  void *const drelu[2], void *xhat_trace, psml_stream stream);
+psml_status psml_secure_relu_fss(psml_ctx ctx, const void *const x[2], int64_t n, const void *const mat[2],
+                                 const void *const U[2], const void *const V[2], const void *const Z[2],
+                                 void *const y[2], void *const drelu[2], psml_stream stream);
+psml_status psml_fss_mask(psml_ctx ctx, int32_t party, const void *x_i, int64_t n, const void *mat_i, void *msg,
+                          psml_stream stream);
+psml_status psml_fss_open_drelu(psml_ctx ctx, int32_t party, const void *msg_send, const void *msg_recv, int64_t n,
+                                const void *mat_i, void *drelu_i, psml_stream stream);
+
 /* Plain ring GEMM C = A . B mod 2^l (A: M x K, B: K x N, row-major) -- the config-5 sweep
  * kernel and the dealer's Z = U V.  Uses the ctx's backend choice. */
 psml_status psml_ring_gemm(psml_ctx ctx, const void *A, const void *B, int64_t M, int64_t K,

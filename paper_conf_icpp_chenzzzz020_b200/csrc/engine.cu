@@ -8,6 +8,7 @@
 #include <vector>
 
 #include "engine.h"
+#include "fss.cuh"
 
 namespace psml {
 
@@ -616,6 +617,121 @@ psml_status psml_secure_eq9(psml_ctx ctx, const void *const x[2], int64_t n, con
     cudaStream_t s = (cudaStream_t)stream;
     if (c->ring.l == 64) return activation_t<uint64_t>(c, 2, x, n, mat, nullptr, nullptr, U, V, Z, y, nullptr, s);
     return activation_t<uint32_t>(c, 2, x, n, mat, nullptr, nullptr, U, V, Z, y, nullptr, s);
+}
+
+// ------------------------------------------------------------------------------------------------
+// one-round FSS comparison (fss.cuh, R22); Z_2^64 only
+// ------------------------------------------------------------------------------------------------
+int64_t psml_fss_material_words(psml_ring ring, int64_t n) {
+    if (ring.l != 64 || n < 0) return -1;
+    return (int64_t)FSS_WORDS * n;
+}
+
+psml_status psml_fss_dealer(psml_ring ring, uint64_t seed, uint64_t call_id, int64_t n, void *const mat[2],
+                            psml_stream stream) {
+    PSML_TRY(check_ring(ring));
+    if (ring.l != 64) return fail(PSML_ERR_UNSUPPORTED, "the FSS comparison is built for Z_2^64");
+    if (n < 0) return fail(PSML_ERR_SHAPE, "n < 0");
+    if (n == 0) return PSML_OK;
+    if (!mat) return fail(PSML_ERR_INVALID, "null pair array");
+    PSML_TRY(check_ptrs({mat[0], mat[1]}));
+    cudaStream_t s = (cudaStream_t)stream;
+    ProfScope prof(PROF_DEALER, s, 2.0 * FSS_BITS * (double)n);
+    fss_dealer_kernel<<<grid_for(n, 128, 148 * 16), 128, 0, s>>>(
+        make_key(seed, TAG_FR, call_id), make_key(seed, TAG_F0, call_id), make_key(seed, TAG_FS, call_id),
+        make_key(seed, TAG_K0, call_id), make_key(seed, TAG_K1, call_id), n, (uint64_t *)mat[0], (uint64_t *)mat[1]);
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
+static psml_status fss_drelu_pair(const void *const x[2], int64_t n, const void *const mat[2], uint64_t *const d[2],
+                                  uint64_t *xhat, uint64_t *ws, cudaStream_t s) {
+    Pair<uint64_t> msg{{ws, ws + n}};
+    {
+        ProfScope prof(PROF_MSB, s, 8.0 * n * 2 * 3);
+        fss_mask_kernel<<<ew_grid(n), EW_THREADS, 0, s>>>(CPair<uint64_t>{{(const uint64_t *)x[0], (const uint64_t *)x[1]}},
+                                                          CPair<uint64_t>{{(const uint64_t *)mat[0], (const uint64_t *)mat[1]}},
+                                                          n, msg, -1);
+        PSML_LAUNCH_CHECK();
+    }
+    ProfScope prof(PROF_MSB, s, 8.0 * n * 2 * (FSS_WORDS + 3));
+    fss_eval_kernel<<<grid_for(2 * n, 128, 148 * 16), 128, 0, s>>>(CPair<uint64_t>{{msg.p[0], msg.p[1]}},
+                                                                  CPair<uint64_t>{{(const uint64_t *)mat[0], (const uint64_t *)mat[1]}},
+                                                                  n, Pair<uint64_t>{{d[0], d[1]}}, xhat, -1);
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
+psml_status psml_secure_drelu_fss(psml_ctx ctx, const void *const x[2], int64_t n, const void *const mat[2],
+                                  void *const drelu[2], void *xhat_trace, psml_stream stream) {
+    if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
+    Ctx *c = reinterpret_cast<Ctx *>(ctx);
+    if (c->ring.l != 64) return fail(PSML_ERR_UNSUPPORTED, "the FSS comparison is built for Z_2^64");
+    if (n < 0) return fail(PSML_ERR_SHAPE, "n < 0");
+    if (n == 0) return PSML_OK;
+    if (!x || !mat || !drelu) return fail(PSML_ERR_INVALID, "null pair array");
+    PSML_TRY(check_ptrs({x[0], x[1], mat[0], mat[1], drelu[0], drelu[1], xhat_trace}));
+    PSML_TRY(c->ensure_ws(sizeof(uint64_t) * 2 * n));
+    uint64_t *d[2] = {(uint64_t *)drelu[0], (uint64_t *)drelu[1]};
+    return fss_drelu_pair(x, n, mat, d, (uint64_t *)xhat_trace, (uint64_t *)c->ws, (cudaStream_t)stream);
+}
+
+psml_status psml_secure_relu_fss(psml_ctx ctx, const void *const x[2], int64_t n, const void *const mat[2],
+                                 const void *const U[2], const void *const V[2], const void *const Z[2],
+                                 void *const y[2], void *const drelu[2], psml_stream stream) {
+    if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
+    Ctx *c = reinterpret_cast<Ctx *>(ctx);
+    if (c->ring.l != 64) return fail(PSML_ERR_UNSUPPORTED, "the FSS comparison is built for Z_2^64");
+    if (n < 0) return fail(PSML_ERR_SHAPE, "n < 0");
+    if (n == 0) return PSML_OK;
+    if (!x || !mat || !U || !V || !Z || !y) return fail(PSML_ERR_INVALID, "null pair array");
+    PSML_TRY(check_ptrs({x[0], x[1], mat[0], mat[1], U[0], U[1], V[0], V[1], Z[0], Z[1], y[0], y[1]}));
+    if (drelu) PSML_TRY(check_ptrs({drelu[0], drelu[1]}));
+    PSML_TRY(c->ensure_ws(sizeof(uint64_t) * 8 * n));
+    uint64_t *ws = (uint64_t *)c->ws;
+    uint64_t *d[2] = {drelu ? (uint64_t *)drelu[0] : ws + 2 * n, drelu ? (uint64_t *)drelu[1] : ws + 3 * n};
+    cudaStream_t s = (cudaStream_t)stream;
+    PSML_TRY(fss_drelu_pair(x, n, mat, d, nullptr, ws, s));
+    const uint64_t *A[2] = {(const uint64_t *)x[0], (const uint64_t *)x[1]};
+    const uint64_t *Bd[2] = {d[0], d[1]};
+    return beaver_hadamard<uint64_t>(A, Bd, (const uint64_t *const *)U, (const uint64_t *const *)V,
+                                     (const uint64_t *const *)Z, n, 0, (uint64_t *const *)y, ws + 4 * n, s);
+}
+
+// split deployment: party `party`'s round-1 message and its evaluation after the exchange
+psml_status psml_fss_mask(psml_ctx ctx, int32_t party, const void *x_i, int64_t n, const void *mat_i, void *msg,
+                          psml_stream stream) {
+    if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
+    if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
+    if (reinterpret_cast<Ctx *>(ctx)->ring.l != 64) return fail(PSML_ERR_UNSUPPORTED, "Z_2^64 only");
+    if (n < 0) return fail(PSML_ERR_SHAPE, "n < 0");
+    if (n == 0) return PSML_OK;
+    PSML_TRY(check_ptrs({x_i, mat_i, msg}));
+    CPair<uint64_t> xx{{nullptr, nullptr}}, mm{{nullptr, nullptr}};
+    Pair<uint64_t> out{{nullptr, nullptr}};
+    xx.p[party] = (const uint64_t *)x_i; mm.p[party] = (const uint64_t *)mat_i; out.p[party] = (uint64_t *)msg;
+    fss_mask_kernel<<<ew_grid(n), EW_THREADS, 0, (cudaStream_t)stream>>>(xx, mm, n, out, party);
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
+psml_status psml_fss_open_drelu(psml_ctx ctx, int32_t party, const void *msg_send, const void *msg_recv, int64_t n,
+                                const void *mat_i, void *drelu_i, psml_stream stream) {
+    if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
+    if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
+    if (reinterpret_cast<Ctx *>(ctx)->ring.l != 64) return fail(PSML_ERR_UNSUPPORTED, "Z_2^64 only");
+    if (n < 0) return fail(PSML_ERR_SHAPE, "n < 0");
+    if (n == 0) return PSML_OK;
+    PSML_TRY(check_ptrs({msg_send, msg_recv, mat_i, drelu_i}));
+    CPair<uint64_t> msg{{nullptr, nullptr}}, mm{{nullptr, nullptr}};
+    msg.p[party] = (const uint64_t *)msg_send;
+    msg.p[1 - party] = (const uint64_t *)msg_recv;
+    mm.p[party] = (const uint64_t *)mat_i;
+    Pair<uint64_t> d{{nullptr, nullptr}};
+    d.p[party] = (uint64_t *)drelu_i;
+    fss_eval_kernel<<<grid_for(n, 128, 148 * 16), 128, 0, (cudaStream_t)stream>>>(msg, mm, n, d, nullptr, party);
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
 }
 
 template <typename T>

@@ -116,6 +116,12 @@ _SIGS = {
     "psml_dp_size": (i32, [vp, vp]),
     "psml_dp_allreduce": (i32, [vp, vp, i64, i32, vp]),
     "psml_party_train_step": (i32, [vp, i32, vp, vp, vp, vp, u32, vp]),
+    "psml_fss_material_words": (i64, [Ring, i64]),
+    "psml_fss_dealer": (i32, [Ring, u64, u64, i64, P2, vp]),
+    "psml_secure_drelu_fss": (i32, [vp, P2, i64, P2, P2, vp, vp]),
+    "psml_secure_relu_fss": (i32, [vp, P2, i64, P2, P2, P2, P2, P2, P2, vp]),
+    "psml_fss_mask": (i32, [vp, i32, vp, i64, vp, vp, vp]),
+    "psml_fss_open_drelu": (i32, [vp, i32, vp, vp, i64, vp, vp, vp]),
     "psml_party_capture_step": (i32, [vp, i32, vp, vp, vp, vp, i32, vp]),
 }
 PEER_HANDLE_BYTES = 256
@@ -413,6 +419,47 @@ def secure_relu(ctx, x, mat, U, V, Z, stream=None):
     _call("psml_secure_relu", ctx.handle, _pair(x), n, _pair(mat), _pair(U), _pair(V), _pair(Z),
           _pair(y), _pair(d), _stream(stream))
     return y, d
+
+
+def fss_dealer(ring, seed, call_id, n, stream=None):
+    """One-round FSS comparison material (psml_fss_dealer, R22): 257 n words per party."""
+    w = lib().psml_fss_material_words(ring, n)
+    if w < 0:
+        raise PsmlError("psml_fss_material_words", 4, "the FSS comparison is built for Z_2^64")
+    mat = empty_pair(w, ring.l)
+    _call("psml_fss_dealer", ring, seed, call_id, n, _pair(mat), _stream(stream))
+    return mat
+
+
+def secure_drelu_fss(ctx, x, mat, trace=False, stream=None):
+    n = x[0].numel()
+    d = empty_pair(x[0].shape, ctx.l)
+    xh = empty(n, ctx.l) if trace else None
+    _call("psml_secure_drelu_fss", ctx.handle, _pair(x), n, _pair(mat), _pair(d), _ptr(xh), _stream(stream))
+    return (d, xh) if trace else d
+
+
+def secure_relu_fss(ctx, x, mat, U, V, Z, stream=None):
+    n = x[0].numel()
+    y, d = empty_pair(x[0].shape, ctx.l), empty_pair(x[0].shape, ctx.l)
+    _call("psml_secure_relu_fss", ctx.handle, _pair(x), n, _pair(mat), _pair(U), _pair(V), _pair(Z),
+          _pair(y), _pair(d), _stream(stream))
+    return y, d
+
+
+def fss_mask(ctx, party, x_i, mat_i, stream=None):
+    n = x_i.numel()
+    msg = empty(n, ctx.l)
+    _call("psml_fss_mask", ctx.handle, party, _ptr(x_i), n, _ptr(mat_i), _ptr(msg), _stream(stream))
+    return msg
+
+
+def fss_open_drelu(ctx, party, msg_send, msg_recv, mat_i, stream=None):
+    n = msg_send.numel()
+    d = empty(n, ctx.l)
+    _call("psml_fss_open_drelu", ctx.handle, party, _ptr(msg_send), _ptr(msg_recv), n, _ptr(mat_i), _ptr(d),
+          _stream(stream))
+    return d
 
 
 def secure_eq9(ctx, x, mat, U, V, Z, stream=None):
