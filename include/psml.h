@@ -292,6 +292,9 @@ typedef struct {
     int32_t fwd_frac_bits[8]; /* per layer f_w (R21): forward weights W = trunc(W^m,
                                  m - f_w), products with W truncated by f_w; 0 = frac_bits.
                                  frac_bits <= f_w <= m.  The CNN config uses {16, 20, 20}.    */
+    int32_t compare;          /* secure comparison of ReLU / Eq. 9: 0 = Kogge-Stone A2B chain +
+                                 daBit (R9, 1 + log2 l + 1 rounds), 1 = one-round FSS
+                                 DCF comparison (R22; material psml_fss_dealer's layout)       */
 } psml_model_desc;
 
 psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_model *out);

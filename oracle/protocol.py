@@ -105,8 +105,9 @@ def sub_pair(a, b):
 class Model:
     """Both parties' weight shares: master (MASTER fractional bits) and forward copy (fw[l] bits)."""
 
-    def __init__(self, task, W_init, fw=None):
+    def __init__(self, task, W_init, fw=None, compare="a2b"):
         self.task = task
+        self.compare = compare   # secure comparison of ReLU / Eq. 9: "a2b" (R9) or "fss" (R22)
         self.fw = list(fw) if fw is not None else list(FWD_BITS[task])
         if task == "mlp" and fw is None:
             self.fw = [F] * len(W_init)
@@ -137,11 +138,17 @@ def matmul(A, B, pair, step, layer, op, trunc):
     return checked_trunc(c, trunc) if trunc else c
 
 
-def relu(z, pair, step, layer):
+def relu(z, pair, step, layer, compare="a2b"):
+    """Secure ReLU: DReLU by the Kogge-Stone A2B chain (R9) or by the one-round FSS comparison
+    (compare="fss", R22: material keyed by the same call id), then one Beaver Hadamard."""
     n = z[0].size
-    mat = core.msb_dealer(DEALER_SEED, call_id(pair, step, layer, OP_RELU_MSB, 0), n, L)
+    cid = call_id(pair, step, layer, OP_RELU_MSB, 0)
     ht = core.hadamard_triplet_gen(DEALER_SEED, call_id(pair, step, layer, OP_HADAMARD, 0), n, L)
-    (r0, r1), (d0, d1) = core.secure_relu((z[0].reshape(-1), z[1].reshape(-1)), mat, ht, L)
+    flat = (z[0].reshape(-1), z[1].reshape(-1))
+    if compare == "fss":
+        (r0, r1), (d0, d1) = core.secure_relu_fss(flat, core.fss_dealer(DEALER_SEED, cid, n, L), ht, L)
+    else:
+        (r0, r1), (d0, d1) = core.secure_relu(flat, core.msb_dealer(DEALER_SEED, cid, n, L), ht, L)
     if DIAG["on"]:   # DReLU = 1 - MSB(x) must equal [x >= 0] on the plaintext
         x = _signed(z[0].reshape(-1) + z[1].reshape(-1))
         dr = np.asarray(d0 + d1, dtype=np.uint64)
@@ -151,11 +158,17 @@ def relu(z, pair, step, layer):
     return (r0.reshape(s), r1.reshape(s)), (d0.reshape(s), d1.reshape(s))
 
 
-def eq9(z, pair, step, layer):
+def eq9(z, pair, step, layer, compare="a2b"):
     n = z[0].size
-    mat = core.msb_dealer(DEALER_SEED, call_id(pair, step, layer, OP_EQ9_MSB, 0), 2 * n, L)
+    cid = call_id(pair, step, layer, OP_EQ9_MSB, 0)
     ht = core.hadamard_triplet_gen(DEALER_SEED, call_id(pair, step, layer, OP_HADAMARD, 2), 2 * n, L)
-    y = core.secure_eq9(z, mat, ht, L, F)
+    if compare == "fss":   # Eq. 9 = ReLU(x + 1/2) - ReLU(x - 1/2) with the FSS ReLU (R22)
+        x = core.eq9_inputs(z, L, F)
+        (r0, r1), _ = core.secure_relu_fss(x, core.fss_dealer(DEALER_SEED, cid, 2 * n, L), ht, L)
+        shape = np.shape(z[0])
+        y = (((r0[:n] - r0[n:]) & MASK).reshape(shape), ((r1[:n] - r1[n:]) & MASK).reshape(shape))
+    else:
+        y = core.secure_eq9(z, core.msb_dealer(DEALER_SEED, cid, 2 * n, L), ht, L, F)
     if DIAG["on"]:   # Eq. 9 on the grid: clamp(x + 2^(F-1), 0, 2^F) exactly (R8)
         x = _signed(z[0] + z[1])
         want = np.clip(x + (1 << (F - 1)), 0, 1 << F)
@@ -223,13 +236,13 @@ def forward_backward(model, Xs, Ys, step, pair=0):
     for layer in range(nl):
         z = matmul(h, model.W[layer], pair, step, layer, OP_FWD, model.fw[layer])
         if layer < nl - 1:
-            h, d = relu(z, pair, step, layer)
+            h, d = relu(z, pair, step, layer, model.compare)
             drelus.append(d)
             acts.append(h)
         elif task == "linreg":
             h = z
         else:
-            h = eq9(z, pair, step, layer)
+            h = eq9(z, pair, step, layer, model.compare)
     yhat = h
     delta = sub_pair(yhat, Ys)
     grads = [None] * nl
@@ -248,12 +261,12 @@ def _cnn_forward_backward(model, Xs, Ys, step, pair):
     # forward conv: V for op 0 is the weight mask (75 x 16), Z = im2col(U) . V
     fw = model.fw
     zc = conv_matmul(Xs, model.W[0], U, V, Z, transpose=False, trunc=fw[0])   # (B*784) x 16
-    h1, d1 = relu(zc, pair, step, 0)
+    h1, d1 = relu(zc, pair, step, 0, model.compare)
     h1 = (h1[0].reshape(B, -1), h1[1].reshape(B, -1))                         # B x 12544
     z2 = matmul(h1, model.W[1], pair, step, 1, OP_FWD, fw[1])
-    h2, d2 = relu(z2, pair, step, 1)
+    h2, d2 = relu(z2, pair, step, 1, model.compare)
     z3 = matmul(h2, model.W[2], pair, step, 2, OP_FWD, fw[2])
-    yhat = eq9(z3, pair, step, 2)
+    yhat = eq9(z3, pair, step, 2, model.compare)
     delta = sub_pair(yhat, Ys)
     grads = [None] * 3
     grads[2] = matmul(_T(h2), delta, pair, step, 2, OP_GRADW, 0)
@@ -295,20 +308,20 @@ def infer(model, Xs, step, pair=0):
         B = Xs[0].shape[0]
         U, V, Z = conv_triplet(pair, step, OP_FWD, B, transpose=False)
         zc = conv_matmul(Xs, model.W[0], U, V, Z, transpose=False, trunc=model.fw[0])
-        h, _ = relu(zc, pair, step, 0)
+        h, _ = relu(zc, pair, step, 0, model.compare)
         h = (h[0].reshape(B, -1), h[1].reshape(B, -1))
         for layer in (1, 2):
             z = matmul(h, model.W[layer], pair, step, layer, OP_FWD, model.fw[layer])
-            h = relu(z, pair, step, layer)[0] if layer == 1 else eq9(z, pair, step, layer)
+            h = relu(z, pair, step, layer, model.compare)[0] if layer == 1 else eq9(z, pair, step, layer, model.compare)
         return h
     h = Xs
     nl = len(model.W)
     for layer in range(nl):
         z = matmul(h, model.W[layer], pair, step, layer, OP_FWD, model.fw[layer])
         if layer < nl - 1:
-            h = relu(z, pair, step, layer)[0]
+            h = relu(z, pair, step, layer, model.compare)[0]
         elif task == "linreg":
             h = z
         else:
-            h = eq9(z, pair, step, layer)
+            h = eq9(z, pair, step, layer, model.compare)
     return h

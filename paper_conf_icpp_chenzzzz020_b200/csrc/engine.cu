@@ -637,29 +637,14 @@ psml_status psml_fss_dealer(psml_ring ring, uint64_t seed, uint64_t call_id, int
     PSML_TRY(check_ptrs({mat[0], mat[1]}));
     cudaStream_t s = (cudaStream_t)stream;
     ProfScope prof(PROF_DEALER, s, 2.0 * FSS_BITS * (double)n);
-    fss_dealer_kernel<<<grid_for(n, 128, 148 * 16), 128, 0, s>>>(
-        make_key(seed, TAG_FR, call_id), make_key(seed, TAG_F0, call_id), make_key(seed, TAG_FS, call_id),
-        make_key(seed, TAG_K0, call_id), make_key(seed, TAG_K1, call_id), n, (uint64_t *)mat[0], (uint64_t *)mat[1]);
-    PSML_LAUNCH_CHECK();
-    return PSML_OK;
+    return fss_dealer_launch(seed, call_id, n, (uint64_t *)mat[0], (uint64_t *)mat[1], s);
 }
 
 static psml_status fss_drelu_pair(const void *const x[2], int64_t n, const void *const mat[2], uint64_t *const d[2],
                                   uint64_t *xhat, uint64_t *ws, cudaStream_t s) {
-    Pair<uint64_t> msg{{ws, ws + n}};
-    {
-        ProfScope prof(PROF_MSB, s, 8.0 * n * 2 * 3);
-        fss_mask_kernel<<<ew_grid(n), EW_THREADS, 0, s>>>(CPair<uint64_t>{{(const uint64_t *)x[0], (const uint64_t *)x[1]}},
-                                                          CPair<uint64_t>{{(const uint64_t *)mat[0], (const uint64_t *)mat[1]}},
-                                                          n, msg, -1);
-        PSML_LAUNCH_CHECK();
-    }
-    ProfScope prof(PROF_MSB, s, 8.0 * n * 2 * (FSS_WORDS + 3));
-    fss_eval_kernel<<<grid_for(2 * n, 128, 148 * 16), 128, 0, s>>>(CPair<uint64_t>{{msg.p[0], msg.p[1]}},
-                                                                  CPair<uint64_t>{{(const uint64_t *)mat[0], (const uint64_t *)mat[1]}},
-                                                                  n, Pair<uint64_t>{{d[0], d[1]}}, xhat, -1);
-    PSML_LAUNCH_CHECK();
-    return PSML_OK;
+    return fss_drelu_launch(CPair<uint64_t>{{(const uint64_t *)x[0], (const uint64_t *)x[1]}}, n,
+                            CPair<uint64_t>{{(const uint64_t *)mat[0], (const uint64_t *)mat[1]}},
+                            Pair<uint64_t>{{d[0], d[1]}}, xhat, ws, s);
 }
 
 psml_status psml_secure_drelu_fss(psml_ctx ctx, const void *const x[2], int64_t n, const void *const mat[2],

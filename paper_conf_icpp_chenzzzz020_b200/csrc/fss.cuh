@@ -15,7 +15,7 @@
 // Streams (R11 keys): r = PRG("FR"), r_0 = PRG("F0"), sA_0 = PRG("FS"), root seeds
 // PRG64("K0")[2e, 2e+1], PRG64("K1")[2e, 2e+1].
 #pragma once
-#include "common.cuh"
+#include "ops.cuh"
 
 namespace psml {
 
@@ -58,7 +58,7 @@ __device__ __forceinline__ void dcf_G(const S128 s, S128 &sL, uint64_t &vL, int 
 __device__ __forceinline__ uint64_t neg_if(int t, uint64_t v) { return t ? (uint64_t)0 - v : v; }
 
 // Dealer (offline): Gen of Fig. 1 for every element; both parties' material.
-__global__ void __launch_bounds__(128) fss_dealer_kernel(PrgKey kr, PrgKey kr0, PrgKey ks0, PrgKey kk0, PrgKey kk1,
+static __global__ void __launch_bounds__(128) fss_dealer_kernel(PrgKey kr, PrgKey kr0, PrgKey ks0, PrgKey kk0, PrgKey kk1,
                                                          int64_t n, uint64_t *__restrict__ mat0,
                                                          uint64_t *__restrict__ mat1) {
     kr = live_key(kr); kr0 = live_key(kr0); ks0 = live_key(ks0); kk0 = live_key(kk0); kk1 = live_key(kk1);
@@ -108,7 +108,7 @@ __global__ void __launch_bounds__(128) fss_dealer_kernel(PrgKey kr, PrgKey kr0, 
 }
 
 // Round 1 (the only opening): party b's message xhat_b = x_b + r_b.  only < 0: both parties.
-__global__ void __launch_bounds__(256) fss_mask_kernel(CPair<uint64_t> x, CPair<uint64_t> mat, int64_t n,
+static __global__ void __launch_bounds__(256) fss_mask_kernel(CPair<uint64_t> x, CPair<uint64_t> mat, int64_t n,
                                                        Pair<uint64_t> msg, int only) {
     for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x)
 #pragma unroll
@@ -118,7 +118,7 @@ __global__ void __launch_bounds__(256) fss_mask_kernel(CPair<uint64_t> x, CPair<
 
 // Open xhat = msg_0 + msg_1, then Eval(b, k_b, xhat') and the local DReLU combination.  One
 // thread per (element, party); xhat_trace (nullable) receives the opened value.
-__global__ void __launch_bounds__(128) fss_eval_kernel(CPair<uint64_t> msg, CPair<uint64_t> mat, int64_t n,
+static __global__ void __launch_bounds__(128) fss_eval_kernel(CPair<uint64_t> msg, CPair<uint64_t> mat, int64_t n,
                                                        Pair<uint64_t> drelu, uint64_t *xhat_trace, int only) {
     const int64_t total = only < 0 ? 2 * n : n;
     for (int64_t g = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; g < total; g += (int64_t)gridDim.x * blockDim.x) {
@@ -157,6 +157,58 @@ __global__ void __launch_bounds__(128) fss_eval_kernel(CPair<uint64_t> msg, CPai
         const uint64_t msb = c ? one - sx : sx;
         drelu.p[b][e] = one - msb;
     }
+}
+
+// Eq. 9 through the FSS ReLU (R22): inputs [z + 1/2 ; z - 1/2] (the public constant added by
+// party 0), and y = r[0, n) - r[n, 2n), delta = y - Y.  only < 0: both parties.
+static __global__ void __launch_bounds__(256) eq9_prep_kernel(CPair<uint64_t> z, int64_t n, uint64_t half,
+                                                              Pair<uint64_t> x, int only) {
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x)
+#pragma unroll
+        for (int p = 0; p < 2; ++p)
+            if (only < 0 || only == p) {
+                const uint64_t h = p == 0 ? half : 0;
+                x.p[p][e] = z.p[p][e] + h;
+                x.p[p][n + e] = z.p[p][e] - h;
+            }
+}
+static __global__ void __launch_bounds__(256) eq9_combine_kernel(CPair<uint64_t> r, int64_t n, Pair<uint64_t> y,
+                                                                 CPair<uint64_t> Y, Pair<uint64_t> delta, int only) {
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x)
+#pragma unroll
+        for (int p = 0; p < 2; ++p)
+            if (only < 0 || only == p) {
+                const uint64_t v = r.p[p][e] - r.p[p][n + e];
+                y.p[p][e] = v;
+                if (delta.p[p]) delta.p[p][e] = v - Y.p[p][e];
+            }
+}
+
+// Dealer launch with keys whose step field may live in device memory (CUDA graphs).
+static inline psml_status fss_dealer_launch(uint64_t seed, uint64_t cid, int64_t n, uint64_t *m0, uint64_t *m1,
+                                            cudaStream_t s, const uint32_t *step = nullptr) {
+    if (n <= 0) return PSML_OK;
+    fss_dealer_kernel<<<grid_for(n, 128, 148 * 16), 128, 0, s>>>(
+        make_key(seed, TAG_FR, cid, step), make_key(seed, TAG_F0, cid, step), make_key(seed, TAG_FS, cid, step),
+        make_key(seed, TAG_K0, cid, step), make_key(seed, TAG_K1, cid, step), n, m0, m1);
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
+// Both parties' DReLU shares: mask round + (open, evaluate).  ws: 2 n words (messages).
+static inline psml_status fss_drelu_launch(CPair<uint64_t> x, int64_t n, CPair<uint64_t> mat, Pair<uint64_t> d,
+                                           uint64_t *xhat, uint64_t *ws, cudaStream_t s) {
+    Pair<uint64_t> msg{{ws, ws + n}};
+    {
+        ProfScope prof(PROF_MSB, s, 8.0 * n * 2 * 3);
+        fss_mask_kernel<<<ew_grid(n), EW_THREADS, 0, s>>>(x, mat, n, msg, -1);
+        PSML_LAUNCH_CHECK();
+    }
+    ProfScope prof(PROF_MSB, s, 8.0 * n * 2 * (FSS_WORDS + 3));
+    fss_eval_kernel<<<grid_for(2 * n, 128, 148 * 16), 128, 0, s>>>(CPair<uint64_t>{{msg.p[0], msg.p[1]}}, mat, n, d,
+                                                                  xhat, -1);
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
 }
 
 }  // namespace psml

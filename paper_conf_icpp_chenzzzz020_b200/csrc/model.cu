@@ -19,13 +19,14 @@
 #include "engine.h"
 #include "dealer_fused.cuh"
 #include "fused.cuh"
+#include "fss.cuh"
 
 namespace psml {
 
 using T = uint64_t;
 
 enum { OP_FWD = 0, OP_GRADW = 1, OP_GRADIN = 2, OP_RELU_MSB = 3, OP_EQ9_MSB = 4, OP_HADAMARD = 6, OP_SHARE = 7 };
-enum ItemKind { IT_MATRIX, IT_CONV_FWD, IT_CONV_GW, IT_HAD, IT_MSB };
+enum ItemKind { IT_MATRIX, IT_CONV_FWD, IT_CONV_GW, IT_HAD, IT_MSB, IT_FSS };   // IT_FSS: DCF material (R22)
 
 __global__ void set_word_kernel(uint32_t *p, uint32_t v) { *p = v; }
 
@@ -99,6 +100,7 @@ struct DealPlan {   // fused dealer of one pool (full or inference-only)
     bool gemm_big = false;   // 64 x 64 tiles, 4 x 4 per thread (ClDealer) instead of ClDefault
     int64_t gemm_tiles = 0;
     std::vector<int> rest;   // items whose Z = U V runs in its own launch (conv, tcgen05-sized)
+    std::vector<int> fss;    // DCF key generation (own launch per item, R22)
 };
 
 }  // namespace psml
@@ -198,7 +200,7 @@ static void add_had(psml_model_s *m, int layer, int slot, int64_t n, bool fwd) {
 }
 static void add_msb(psml_model_s *m, int layer, int op, int64_t n, bool fwd) {
     DealItem it;
-    it.kind = IT_MSB; it.layer = layer; it.op = op; it.slot = 0; it.n = n; it.fwd = fwd;
+    it.kind = m->d.compare == 1 ? IT_FSS : IT_MSB;   // comparison material: A2B chain (R9) or DCF (R22) it.layer = layer; it.op = op; it.slot = 0; it.n = n; it.fwd = fwd;
     m->items[0].push_back(it);
 }
 
@@ -285,6 +287,9 @@ static psml_status alloc_items(psml_model_s *m, std::vector<DealItem> &items) {
         case IT_MSB:
             PSML_TRY(balloc(m, it.mat, psml_msb_material_words(ring, it.n)));
             break;
+        case IT_FSS:
+            PSML_TRY(balloc(m, it.mat, (int64_t)FSS_WORDS * it.n));
+            break;
         }
     }
     return PSML_OK;
@@ -303,6 +308,7 @@ static int64_t ws_need(psml_model_s *m) {
         case IT_CONV_GW: w = std::max(w, conv_ws_words<T>(m->B, m->g, 1, it.N)); break;
         case IT_HAD: w = std::max(w, 4 * it.n); break;
         case IT_MSB: w = std::max(w, msb_ws_words<T>(it.n)); break;
+        case IT_FSS: w = std::max(w, 12 * it.n); break;
         }
     }
     return w;
@@ -311,7 +317,7 @@ static int64_t ws_need(psml_model_s *m) {
 static int64_t dws_need(psml_model_s *m) {
     int64_t w = 1;   // dealer: split-K partials of the Z = U V GEMMs (or the tcgen05 limb planes)
     for (auto &it : m->items[0]) {
-        if (it.kind != IT_HAD && it.kind != IT_MSB) w = std::max(w, it.M * it.N);
+        if (it.kind != IT_HAD && it.kind != IT_MSB && it.kind != IT_FSS) w = std::max(w, it.M * it.N);
         if (it.kind == IT_MATRIX && m->ctx->use_tc(it.M, it.K, it.N))
             w = std::max(w, (int64_t)(tc_ring_gemm_ws_bytes(64, it.M, it.K, it.N) + 7) / 8);
     }
@@ -376,6 +382,10 @@ static psml_status deal_item(psml_model_s *m, DealItem &it, uint32_t step, cudaS
         ProfScope prof(PROF_DEALER, s, (double)sizeof(T) * 2 * it.mat.n);
         void *mt[2] = {it.mat.p[0], it.mat.p[1]};
         return msb_dealer_launch<T>(seed, cid, it.n, mt, s, m->step_dev);
+    }
+    case IT_FSS: {
+        ProfScope prof(PROF_DEALER, s, 2.0 * FSS_BITS * (double)it.n);
+        return fss_dealer_launch(seed, cid, it.n, it.mat.p[0], it.mat.p[1], s, m->step_dev);
     }
     }
     return PSML_OK;
@@ -451,6 +461,9 @@ static psml_status build_plan(psml_model_s *m, int pool, bool infer_only) {
             job(PJ_DABIT, {TAG_R0, TAG_R1, TAG_RA}, cid, n, {m0 + o, m1 + o, m0 + o + n, m1 + o + n});
             break;
         }
+        case IT_FSS:
+            P.fss.push_back((int)k);
+            break;
         }
     }
     std::vector<PrgJob> pj(pjm);
@@ -563,6 +576,7 @@ static psml_status deal_pool(psml_model_s *m, int pool, uint32_t step, bool infe
         }
     }
     for (int k : P.rest) PSML_TRY(deal_gemm(m, m->items[pool][k], s));
+    for (int k : P.fss) PSML_TRY(deal_item(m, m->items[pool][k], 0, s));   // step from m->step_dev
     if (fork) PSML_CUDA_TRY(cudaStreamWaitEvent(s, m->ev_d2j, 0));
     return PSML_OK;
 }
@@ -584,10 +598,22 @@ static psml_status mm(psml_model_s *m, const T *const A[2], const T *const Bm[2]
                             m->ws_words, s, m->ctx->sm_count);
 }
 
+// FSS ReLU (R22) of n elements, both parties: DReLU from one opening, then the Beaver Hadamard.
+// ws: 8 n words.
+static psml_status relu_fss(const T *const x[2], int64_t n, const DealItem *mat, const DealItem *h, T *const y[2],
+                            T *const dr[2], T *ws, cudaStream_t s) {
+    T *d[2] = {dr ? dr[0] : ws + 2 * n, dr ? dr[1] : ws + 3 * n};
+    PSML_TRY(fss_drelu_launch(CPair<T>{{x[0], x[1]}}, n, CPair<T>{{mat->mat.p[0], mat->mat.p[1]}}, Pair<T>{{d[0], d[1]}},
+                              nullptr, ws, s));
+    const T *dc[2] = {d[0], d[1]};
+    return beaver_hadamard<T>(x, dc, h->U.cp(), h->V.cp(), h->Z.cp(), n, 0, y, ws + 4 * n, s);
+}
+
 static psml_status relu(psml_model_s *m, const T *const x[2], int layer, T *const y[2], T *const dr[2],
                         cudaStream_t s) {
     DealItem *mat = find_item(m, layer, OP_RELU_MSB, 0), *h = find_item(m, layer, OP_HADAMARD, 0);
     if (!mat || !h) return fail(PSML_ERR_STATE, "missing ReLU material");
+    if (mat->kind == IT_FSS) return relu_fss(x, mat->n, mat, h, y, dr, m->ws, s);
     return msb_chain<T>(x, mat->n, mat->mat.cp(), 0, 0, 1, nullptr, nullptr, dr, h->U.cp(), h->V.cp(), h->Z.cp(), y,
                         nullptr, nullptr, m->ws, s);
 }
@@ -597,6 +623,19 @@ static psml_status eq9(psml_model_s *m, const T *const z[2], int layer, T *const
     DealItem *mat = find_item(m, layer, OP_EQ9_MSB, 0), *h = find_item(m, layer, OP_HADAMARD, 2);
     if (!mat || !h) return fail(PSML_ERR_STATE, "missing Eq. 9 material");
     const T half = (T)1 << (m->ctx->ring.frac_bits - 1);
+    if (mat->kind == IT_FSS) {   // Eq. 9 = ReLU(z + 1/2) - ReLU(z - 1/2) with the FSS ReLU (R22)
+        const int64_t n2 = mat->n, n = n2 / 2;
+        T *xin[2] = {m->ws + 8 * n2, m->ws + 9 * n2}, *r[2] = {m->ws + 10 * n2, m->ws + 11 * n2};
+        eq9_prep_kernel<<<ew_grid(n), EW_THREADS, 0, s>>>(CPair<T>{{z[0], z[1]}}, n, half, Pair<T>{{xin[0], xin[1]}}, -1);
+        PSML_LAUNCH_CHECK();
+        const T *xc[2] = {xin[0], xin[1]};
+        PSML_TRY(relu_fss(xc, n2, mat, h, r, nullptr, m->ws, s));
+        eq9_combine_kernel<<<ew_grid(n), EW_THREADS, 0, s>>>(CPair<T>{{r[0], r[1]}}, n, Pair<T>{{y[0], y[1]}},
+                                                              CPair<T>{{Y ? Y[0] : nullptr, Y ? Y[1] : nullptr}},
+                                                              Pair<T>{{dlt ? dlt[0] : nullptr, dlt ? dlt[1] : nullptr}}, -1);
+        PSML_LAUNCH_CHECK();
+        return PSML_OK;
+    }
     return msb_chain<T>(z, mat->n, mat->mat.cp(), 1, half, 2, nullptr, nullptr, nullptr, h->U.cp(), h->V.cp(),
                         h->Z.cp(), y, Y, dlt, m->ws, s);
 }
@@ -702,6 +741,7 @@ static bool fused_eligible(const psml_model_s *m) {
     if (m->d.kind == PSML_CNN || m->nl > UPD_MAX_LAYERS || (int)m->ob.size() != (int)m->items[0].size()) return false;
     for (int l = 0; l < m->nl; ++l)
         if (fw(m, l) != m->ctx->ring.frac_bits) return false;   // the fused step truncates by F
+    if (m->d.compare != 0) return false;                         // the fused step runs the A2B chain
     return fuse_enabled() && chain_mode() == 0;
 }
 
@@ -988,10 +1028,66 @@ static psml_status party_mm(PartyRun &r, const T *A, const T *Bm, int layer, int
                                    C, ps);
 }
 
+// FSS comparison (R22), one party: round 1 exchanges x_i + r_i, the DCF evaluation gives DReLU,
+// round 2 is the Beaver Hadamard x . DReLU.  what 1 = ReLU, 2 = Eq. 9 (x = z of n/2 elements).
+static psml_status party_chain_fss(PartyRun &r, const T *x, const DealItem *mat, const DealItem *h, int what, T *y,
+                                   T *drelu, const T *Ysub, T *delta) {
+    psml_model_s *m = r.m;
+    const int p = r.p, q = 1 - p;
+    const int64_t n = mat->n;
+    T *ws = m->ws;
+    T *xin = ws, *d = ws + 3 * n, *rr = ws + 8 * n;
+    Pair<T> msg{{nullptr, nullptr}}, mE{{nullptr, nullptr}}, mF{{nullptr, nullptr}};
+    msg.p[p] = ws + n; msg.p[q] = ws + 2 * n;
+    mE.p[p] = ws + 4 * n; mE.p[q] = ws + 5 * n;
+    mF.p[p] = ws + 6 * n; mF.p[q] = ws + 7 * n;
+    const T *xe = x;
+    if (what == 2) {
+        const T half = (T)1 << (m->ctx->ring.frac_bits - 1);
+        eq9_prep_kernel<<<ew_grid(n / 2), EW_THREADS, 0, r.s>>>(mine_c(p, x), n / 2, half, mine(p, xin), p);
+        PSML_LAUNCH_CHECK();
+        xe = xin;
+    }
+    if (what == 1 && drelu) d = drelu;
+    {
+        ProfScope prof(PROF_MSB, r.s, 0.0);
+        fss_mask_kernel<<<ew_grid(n), EW_THREADS, 0, r.s>>>(mine_c(p, xe), mine_c(p, mat->mat.p[p]), n, msg, p);
+        PSML_LAUNCH_CHECK();
+    }
+    PSML_TRY(xchg(r, {{msg.p[p], msg.p[q], n}}));   // the only opening of the comparison: xhat
+    {
+        ProfScope prof(PROF_MSB, r.s, 0.0);
+        fss_eval_kernel<<<grid_for(n, 128, 148 * 16), 128, 0, r.s>>>(CPair<T>{{msg.p[0], msg.p[1]}},
+                                                                    mine_c(p, mat->mat.p[p]), n, mine(p, d), nullptr, p);
+        PSML_LAUNCH_CHECK();
+    }
+    const T *U = h->U.p[p], *V = h->V.p[p], *Z = h->Z.p[p];
+    {
+        ProfScope prof(PROF_HAD, r.s, 0.0);
+        hadamard_mask_kernel<T><<<ew_grid(n), EW_THREADS, 0, r.s>>>(mine_c(p, xe), mine_c(p, d), mine_c(p, U),
+                                                                    mine_c(p, V), n, mE, mF, p);
+        PSML_LAUNCH_CHECK();
+    }
+    PSML_TRY(xchg(r, {{mE.p[p], mE.p[q], n}, {mF.p[p], mF.p[q], n}}));
+    ProfScope prof(PROF_HAD, r.s, 0.0);
+    CPair<T> ce{{mE.p[0], mE.p[1]}}, cf{{mF.p[0], mF.p[1]}};
+    hadamard_open_kernel<T><<<ew_grid(n), EW_THREADS, 0, r.s>>>(ce, cf, mine_c(p, U), mine_c(p, V), mine_c(p, Z), n, 0,
+                                                               mine(p, what == 2 ? rr : y), p);
+    PSML_LAUNCH_CHECK();
+    if (what == 2) {
+        Pair<T> dl{{nullptr, nullptr}};
+        if (delta) dl.p[p] = delta;
+        eq9_combine_kernel<<<ew_grid(n / 2), EW_THREADS, 0, r.s>>>(mine_c(p, rr), n / 2, mine(p, y), mine_c(p, Ysub), dl, p);
+        PSML_LAUNCH_CHECK();
+    }
+    return PSML_OK;
+}
+
 // MSB chain, one round per kernel with an exchange after each (R9):
 // what 1 = ReLU (y = x . drelu, drelu kept), 2 = Eq. 9 (x = z of n/2; y, delta = y - Ysub).
 static psml_status party_chain(PartyRun &r, const T *x, const DealItem *mat, const DealItem *h, int what, T *y,
                                T *drelu, const T *Ysub, T *delta) {
+    if (mat->kind == IT_FSS) return party_chain_fss(r, x, mat, h, what, y, drelu, Ysub, delta);
     psml_model_s *m = r.m;
     const int p = r.p, q = 1 - p;
     const int64_t n = mat->n;

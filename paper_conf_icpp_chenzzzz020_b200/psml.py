@@ -44,7 +44,7 @@ class ModelDesc(ctypes.Structure):
                 ("lr_shift", i32), ("master_frac_bits", i32), ("dealer_seed", u64),
                 ("pair_id", u32), ("cnn_c", i32), ("cnn_h", i32), ("cnn_w", i32), ("cnn_k", i32),
                 ("cnn_cout", i32), ("cnn_hidden", i32), ("cnn_classes", i32),
-                ("fwd_frac_bits", i32 * 8)]
+                ("fwd_frac_bits", i32 * 8), ("compare", i32)]
 
 
 # psml_exchange_fn (include/psml.h): (user, n, send[], recv[], bytes[], stream) -> 0 on success
@@ -514,7 +514,7 @@ class Model:
 
     def __init__(self, ctx, kind, dims=None, batch=128, lr_shift=14, master_frac_bits=27,
                  dealer_seed=0x50534D4C + 2, pair_id=0, cnn=(3, 32, 32, 5, 16, 64, 10),
-                 fwd_frac_bits=None):
+                 fwd_frac_bits=None, compare=0):
         d = ModelDesc()
         d.kind = kind
         dims = list(dims or ([784, 1] if kind in (LINREG, LOGREG) else [784, 128, 128, 10]))
@@ -526,6 +526,7 @@ class Model:
         (d.cnn_c, d.cnn_h, d.cnn_w, d.cnn_k, d.cnn_cout, d.cnn_hidden, d.cnn_classes) = cnn
         for i, v in enumerate(fwd_frac_bits or []):   # per-layer forward-weight bits (R21)
             d.fwd_frac_bits[i] = v
+        d.compare = compare                           # 0 A2B chain (R9), 1 FSS comparison (R22)
         self.ctx, self.desc, self.kind = ctx, d, kind
         h = vp()
         _call("psml_model_create", ctx.handle, ctypes.byref(d), ctypes.byref(h))

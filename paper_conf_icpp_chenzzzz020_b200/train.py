@@ -37,7 +37,7 @@ class SecureTrainer:
     """One co-resident party pair on the current GPU, training `task` with batch `batch`."""
 
     def __init__(self, task, W_init, batch=128, pair_id=0, dims=None, backend=0,
-                 frac_bits=13, master_frac_bits=27, lr_shift=14):
+                 frac_bits=13, master_frac_bits=27, lr_shift=14, compare="a2b"):
         self.task = task
         self.ctx = psml.Ctx(l=64, frac_bits=frac_bits, backend=backend)
         self.ring = self.ctx.ring
@@ -46,7 +46,8 @@ class SecureTrainer:
         self.batch = batch
         self.model = psml.Model(self.ctx, KINDS[task], dims=dims, batch=batch, lr_shift=lr_shift,
                                 master_frac_bits=master_frac_bits, dealer_seed=DEALER_SEED,
-                                pair_id=pair_id, fwd_frac_bits=FWD_BITS.get(task))
+                                pair_id=pair_id, fwd_frac_bits=FWD_BITS.get(task),
+                                compare={"a2b": 0, "fss": 1}[compare])
         for layer, W in enumerate(W_init):
             w = psml.encode(self.master_ring, torch.as_tensor(W, dtype=torch.float64))
             Wm = psml.share(self.ring, SHARE_SEED, call_id(0, INIT_STEP, layer, OP_SHARE, 2), w)

@@ -75,3 +75,37 @@ def test_fss_relu_bitexact_and_split_form(P, orc, ctx, n):
     dd = [P.fss_open_drelu(ctx, p, msgs[p], msgs[1 - p], _dev(mat[p])) for p in range(2)]
     torch.cuda.synchronize()
     assert np.array_equal(to_np(dd[0]), d0) and np.array_equal(to_np(dd[1]), d1)
+
+
+# --- the FSS comparison inside training (psml_model_desc.compare = 1) ------------------------------
+def _compare_shares(tr, om):
+    for layer in range(len(om.Wm)):
+        g0, g1 = tr.master_shares(layer)
+        assert np.array_equal(to_np(g0).reshape(om.Wm[layer][0].shape), om.Wm[layer][0]), layer
+        assert np.array_equal(to_np(g1).reshape(om.Wm[layer][1].shape), om.Wm[layer][1]), layer
+
+
+@pytest.mark.parametrize("task,steps", [("logreg", 2), ("mlp", 2)])
+def test_training_with_fss_comparison_bitexact(P, task, steps):
+    """Every ReLU / Eq. 9 of the step through the one-round FSS comparison: eager steps and
+    CUDA-graph replays (dealer inside the graph) bit-exact vs the oracle's protocol."""
+    import synth
+    from oracle import protocol as OP
+    from paper_conf_icpp_chenzzzz020_b200.train import SecureTrainer
+    Wi = synth.init_weights(task)
+    tr = SecureTrainer(task, Wi, backend=1, compare="fss")
+    om = OP.Model(task, Wi, compare="fss")
+    X, Y = synth.batch(task, 0)
+    tr.step(torch.from_numpy(X), torch.from_numpy(Y), 0)
+    OP.train_step(om, X, Y, 0)
+    torch.cuda.synchronize()
+    _compare_shares(tr, om)
+    if steps > 1:
+        tr.capture(pipelined=True)
+        for s in range(1, steps + 1):
+            X, Y = synth.batch(task, s)
+            tr.graph_step(torch.from_numpy(X), torch.from_numpy(Y), s)
+            OP.train_step(om, X, Y, s)
+            torch.cuda.synchronize()
+            _compare_shares(tr, om)
+    tr.close()

@@ -120,9 +120,10 @@ def test_split_compressed_transmission(tmp_path):
 # must equal the oracle's simulation of both parties (oracle/protocol.py) after every step.
 # ---------------------------------------------------------------------------------------------
 SPLIT_TASKS = [("linreg", 2), ("logreg", 2), ("mlp", 2), ("cnn", 1)]
+FSS_TASKS = [("logreg", 2), ("mlp", 2)]
 
 
-def _party_train(rank, port, outdir, kind):
+def _party_train(rank, port, outdir, kind, compare="a2b"):
     import sys
     sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
     import synth
@@ -133,8 +134,8 @@ def _party_train(rank, port, outdir, kind):
     torch.cuda.set_device(0)
     xp = make_transport(rank, 1 - rank, kind=kind)
     dp = make_dp([rank], rank)          # one pair: the party's data-parallel group is itself
-    for task, steps in SPLIT_TASKS:
-        tr = PartyTrainer(task, synth.init_weights(task), rank, xp, backend=1, dp=dp)
+    for task, steps in (SPLIT_TASKS if compare == "a2b" else FSS_TASKS):
+        tr = PartyTrainer(task, synth.init_weights(task), rank, xp, backend=1, dp=dp, compare=compare)
         for s in range(steps):
             X, Y = synth.batch(task, s)
             tr.step(torch.from_numpy(X), torch.from_numpy(Y), s)
@@ -150,11 +151,11 @@ def _party_train(rank, port, outdir, kind):
     dist.destroy_process_group()
 
 
-def _check_against_oracle(tmp_path, tasks):
+def _check_against_oracle(tmp_path, tasks, compare="a2b"):
     import synth
     from oracle import protocol as OP
     for task, steps in tasks:
-        om = OP.Model(task, synth.init_weights(task))
+        om = OP.Model(task, synth.init_weights(task), compare=compare)
         for s in range(steps):
             X, Y = synth.batch(task, s)
             OP.train_step(om, X, Y, s)
@@ -174,6 +175,15 @@ def test_split_training_matches_oracle(tmp_path, kind):
     _check_against_oracle(tmp_path, SPLIT_TASKS)
     st = [np.load(tmp_path / f"xstats_{p}.npy") for p in range(2)]
     assert st[0][1] == st[1][1] > 0 and st[0][0] == st[1][0] > 0   # symmetric exchanges
+
+
+def test_split_training_fss_comparison_matches_oracle(tmp_path):
+    """The split step with the one-round FSS comparison (R22): per ReLU / Eq. 9 one exchange of
+    x_i + r_i and one Hadamard E/F exchange instead of 9 rounds; bit-exact vs the oracle."""
+    mp.spawn(_party_train, args=(_free_port(), str(tmp_path), "peer", "fss"), nprocs=2, join=True)
+    _check_against_oracle(tmp_path, FSS_TASKS, compare="fss")
+    st = [np.load(tmp_path / f"xstats_{p}.npy") for p in range(2)]
+    assert st[0][1] == st[1][1] > 0
 
 
 GRAPH_TASKS = [("mlp", 4), ("logreg", 3)]

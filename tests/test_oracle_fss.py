@@ -87,3 +87,26 @@ def test_secure_relu_fss_matches_a2b_relu(orc):
     (a0, a1), _ = orc.secure_relu(xs, orc.msb_dealer(15, 1, n), ht)
     assert np.array_equal(r0 + r1, a0 + a1)
     assert np.array_equal(r0 + r1, np.where(_signed(x, 64) >= 0, x, np.uint64(0)).astype(np.uint64))
+
+
+@pytest.mark.parametrize("task,steps,tol_log2", [("logreg", 30, -16), ("mlp", 4, -15)])
+def test_training_with_fss_comparison_tracks_fp64(task, steps, tol_log2):
+    """The protocol with every ReLU / Eq. 9 comparison done by the one-round FSS DReLU (R22):
+    decoded master weights vs fp64 SGD, and zero comparison mismatches / truncation failures."""
+    import synth
+    from oracle import plain
+    from oracle import protocol as P
+    Wi = synth.init_weights(task)
+    m, pm = P.Model(task, Wi, compare="fss"), plain.PlainModel(task, Wi)
+    P.diag_reset(True)
+    try:
+        for s in range(steps):
+            X, Y = synth.batch(task, s)
+            P.train_step(m, X, Y, s)
+            pm.step(X, Y)
+        d = dict(P.DIAG)
+    finally:
+        P.diag_reset(False)
+    assert d["msb_checked"] > 0 and d["msb_fail"] == 0 and d["trunc_fail"] == 0, d
+    err = max(np.abs(a - b).max() for a, b in zip(m.decoded_master(), pm.W))
+    assert err < 2.0 ** tol_log2, np.log2(err)
