@@ -200,7 +200,8 @@ static void add_had(psml_model_s *m, int layer, int slot, int64_t n, bool fwd) {
 }
 static void add_msb(psml_model_s *m, int layer, int op, int64_t n, bool fwd) {
     DealItem it;
-    it.kind = m->d.compare == 1 ? IT_FSS : IT_MSB;   // comparison material: A2B chain (R9) or DCF (R22) it.layer = layer; it.op = op; it.slot = 0; it.n = n; it.fwd = fwd;
+    it.kind = m->d.compare == 1 ? IT_FSS : IT_MSB;   // comparison material: A2B chain (R9) or DCF (R22)
+    it.layer = layer; it.op = op; it.slot = 0; it.n = n; it.fwd = fwd;
     m->items[0].push_back(it);
 }
 
