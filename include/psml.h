@@ -277,11 +277,15 @@ psml_status psml_delta_apply(psml_ctx ctx, int64_t rows, int64_t cols, int32_t i
 /* ------------------------------------------------------------------------------------------ */
 /* Models: secure training / inference (Sec. 4.3, Sec. 7.1)      */
 /* ------------------------------------------------------------------------------------------ */
-typedef enum { PSML_LINREG = 0, PSML_LOGREG = 1, PSML_MLP = 2, PSML_CNN = 3 } psml_model_kind;
+/* PSML_SVM: linear SVM, hinge-loss minibatch subgradient with weight decay (PAPER.md L295 names
+ * SVM trained by SMO; R24 reads it as the primal subgradient form that runs on the
+ * Beaver / comparison primitives): z = X w; ind = [y z < 1]; gradW = X^T (-(y (.) ind)); labels
+ * +-1.  Co-resident engine only. */
+typedef enum { PSML_LINREG = 0, PSML_LOGREG = 1, PSML_MLP = 2, PSML_CNN = 3, PSML_SVM = 4 } psml_model_kind;
 
 typedef struct {
     int32_t kind;             /* psml_model_kind                                             */
-    int32_t n_layers;         /* LINREG/LOGREG: 1; MLP: len(dims)-1; CNN: 3                  */
+    int32_t n_layers;         /* LINREG/LOGREG/SVM: 1; MLP: len(dims)-1; CNN: 3              */
     int64_t dims[8];          /* MLP: layer widths d_0..d_L; LINREG/LOGREG: {784, 1}         */
     int32_t batch;            /* rows per step per pair (128)                                */
     int32_t lr_shift;         /* eta/|B| = 2^-lr_shift (14)                                  */
@@ -295,6 +299,8 @@ typedef struct {
     int32_t compare;          /* secure comparison of ReLU / Eq. 9: 0 = Kogge-Stone A2B chain +
                                  daBit (R9, 1 + log2 l + 1 rounds), 1 = one-round FSS
                                  DCF comparison (R22; material psml_fss_dealer's layout)       */
+    int32_t weight_decay_shift; /* 0 = none; else W^m -= trunc(W^m, shift) every update (SVM:
+                                   lambda.eta = 2^-16, R24)                        */
 } psml_model_desc;
 
 psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_model *out);

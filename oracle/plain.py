@@ -12,7 +12,7 @@ only differences from the secure run are fixed-point rounding and truncation noi
 """
 import numpy as np
 
-from .protocol import F, LR_SHIFT, MASTER, CNN_GEOM
+from .protocol import F, LR_SHIFT, MASTER, CNN_GEOM, WD_SHIFT
 
 
 def q(x, f):
@@ -55,7 +55,7 @@ class PlainModel:
         self.W = [q(W, MASTER) for W in W_init]
 
     def forward(self, X):
-        if self.task == "linreg":
+        if self.task in ("linreg", "svm"):
             return [X], [], X @ self.W[0]
         if self.task == "logreg":
             return [X], [], eq9(X @ self.W[0])
@@ -83,6 +83,11 @@ class PlainModel:
     def step(self, X, Y):
         X, Y = q(X, F), q(Y, F)
         acts, masks, yhat = self.forward(X)
+        if self.task == "svm":   # hinge subgradient + weight decay (R24)
+            delta = -Y * ((Y * yhat) < 1.0)
+            g = X.T @ delta
+            self.W[0] = self.W[0] - 2.0 ** -LR_SHIFT * g - 2.0 ** -WD_SHIFT * self.W[0]
+            return yhat
         delta = yhat - Y
         lr = 2.0 ** -LR_SHIFT
         grads = [None] * len(self.W)

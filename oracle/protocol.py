@@ -37,7 +37,9 @@ CNN_GEOM = dict(C=3, H=32, W=32, k=5, Cout=16, hidden=64, classes=10)
 # h.W and backprop delta.W^T) is truncated by f_w, so activations and deltas stay at F = 13 bits.
 # f_w = F except the CNN, whose 12544-wide FC1 and 5x5 conv fail BJ's 2^-12 weight bound at
 # f_w = 13 (weights of magnitude ~0.005 quantised at 2^-13 perturb every pre-activation).
-FWD_BITS = {"linreg": [F], "logreg": [F], "mlp": [F, F, F], "cnn": [16, 20, 20]}
+FWD_BITS = {"linreg": [F], "logreg": [F], "svm": [F], "mlp": [F, F, F], "cnn": [16, 20, 20]}
+# linear SVM (R24): weight decay lambda.eta = 2^-WD_SHIFT applied to the master weights
+WD_SHIFT = 16
 
 
 def call_id(pair, step, layer, op, slot=0):
@@ -46,7 +48,7 @@ def call_id(pair, step, layer, op, slot=0):
 
 
 def dims_of(task):
-    return {"linreg": [784, 1], "logreg": [784, 1], "mlp": [784, 128, 128, 10],
+    return {"linreg": [784, 1], "logreg": [784, 1], "svm": [784, 1], "mlp": [784, 128, 128, 10],
             "cnn": [None, 12544, 64, 10]}[task]
 
 
@@ -224,11 +226,45 @@ def conv_matmul(X, Bm, U, V, Z, transpose, trunc):
 # ---------------------------------------------------------------------------------------------
 # training step
 # ---------------------------------------------------------------------------------------------
+def comparison_lt0(t, pair, step, layer, compare="a2b"):
+    """Arithmetic shares of [t < 0] (signed) = MSB(t): the A2B chain's MSB (R9), or 1 - DReLU from
+    the FSS comparison (R22).  Material keyed like ReLU's (op 3)."""
+    n = t[0].size
+    cid = call_id(pair, step, layer, OP_RELU_MSB, 0)
+    flat = (t[0].reshape(-1), t[1].reshape(-1))
+    if compare == "fss":
+        d0, d1 = core.fss_drelu(flat, core.fss_dealer(DEALER_SEED, cid, n, L), L)
+        out = ((np.uint64(1) - d0) & MASK, (np.uint64(0) - d1) & MASK)
+    else:
+        out = core.secure_msb(flat, core.msb_dealer(DEALER_SEED, cid, n, L), L)
+    if DIAG["on"]:
+        x = _signed(flat[0] + flat[1])
+        DIAG["msb_checked"] += int(x.size)
+        DIAG["msb_fail"] += int(np.count_nonzero((out[0] + out[1]) != (x < 0).astype(np.uint64)))
+    s = t[0].shape
+    return out[0].reshape(s), out[1].reshape(s)
+
+
+def _svm_forward_backward(model, Xs, Ys, step, pair):
+    """Linear SVM, hinge loss, minibatch subgradient (R24; PAPER.md L295 names SVM):
+    z = X w;  m = y (.) z;  ind = [m < 1] = [m - 1 < 0];  delta = -(y (.) ind);  gradW = X^T delta."""
+    z = matmul(Xs, model.W[0], pair, step, 0, OP_FWD, model.fw[0])
+    m = checked_trunc(hadamard(Ys, z, pair, step, 0, 3), F)            # margin, 13 bits
+    t = ((m[0] - np.uint64(1 << F)) & MASK, m[1])                       # m - 1 (party 0)
+    ind = comparison_lt0(t, pair, step, 0, model.compare)
+    c = hadamard(Ys, ind, pair, step, 0, 4)                             # y (.) ind, 13 bits
+    delta = ((np.uint64(0) - c[0]) & MASK, (np.uint64(0) - c[1]) & MASK)
+    grads = [matmul(_T(Xs), delta, pair, step, 0, OP_GRADW, 0)]
+    return grads, z
+
+
 def forward_backward(model, Xs, Ys, step, pair=0):
     """Returns (per-layer untruncated weight-gradient shares, prediction shares)."""
     task = model.task
     if task == "cnn":
         return _cnn_forward_backward(model, Xs, Ys, step, pair)
+    if task == "svm":
+        return _svm_forward_backward(model, Xs, Ys, step, pair)
     nl = len(model.W)
     acts = [Xs]
     drelus = []
@@ -290,6 +326,8 @@ def apply_update(model, grads, n_pairs=1):
     assert (1 << extra) == n_pairs
     for layer, g in enumerate(grads):
         gt = checked_trunc(g, 2 * F + LR_SHIFT - MASTER + extra)
+        if model.task == "svm":   # weight decay: W^m -= trunc(W^m, WD_SHIFT) (R24), from the old W^m
+            gt = (gt[0] + trunc_pair(model.Wm[layer], WD_SHIFT)[0], gt[1] + trunc_pair(model.Wm[layer], WD_SHIFT)[1])
         model.Wm[layer] = sub_pair(model.Wm[layer], gt)
         model.W[layer] = checked_trunc(model.Wm[layer], MASTER - model.fw[layer])
 
@@ -320,7 +358,7 @@ def infer(model, Xs, step, pair=0):
         z = matmul(h, model.W[layer], pair, step, layer, OP_FWD, model.fw[layer])
         if layer < nl - 1:
             h = relu(z, pair, step, layer, model.compare)[0]
-        elif task == "linreg":
+        elif task in ("linreg", "svm"):   # SVM inference: w^T x
             h = z
         else:
             h = eq9(z, pair, step, layer, model.compare)

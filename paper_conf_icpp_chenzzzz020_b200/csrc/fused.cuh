@@ -166,6 +166,7 @@ struct UpdateAll {
     const T *g[UPD_MAX_LAYERS][2];
     int64_t begin[UPD_MAX_LAYERS + 1];
     int nl, s_grad, s_fwd[UPD_MAX_LAYERS];
+    int wd;   // weight-decay shift (0 = none; SVM, R24)
 };
 
 template <typename T>
@@ -180,7 +181,9 @@ __global__ void __launch_bounds__(256) update_all_kernel(const __grid_constant__
         const int64_t i = x - u.begin[l];
 #pragma unroll
         for (int p = 0; p < 2; ++p) {
-            const T wm = u.Wm[l][p][i] - trunc_share<T>(u.g[l][p][i], p, u.s_grad);
+            const T old = u.Wm[l][p][i];
+            const T dec = u.wd ? trunc_share<T>(old, p, u.wd) : (T)0;
+            const T wm = old - (trunc_share<T>(u.g[l][p][i], p, u.s_grad) + dec);
             u.Wm[l][p][i] = wm;
             u.W[l][p][i] = trunc_share<T>(wm, p, u.s_fwd[l]);
         }

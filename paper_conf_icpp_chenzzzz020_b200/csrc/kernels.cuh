@@ -688,14 +688,18 @@ __global__ void sub_pair_kernel(CPair<T> a, CPair<T> b, int64_t n, Pair<T> c, in
     }
 }
 
-// W^m_i -= trunc_i(g_i, s_grad); W_i = trunc_i(W^m_i, s_fwd)   (R14)
+// W^m_i -= trunc_i(g_i, s_grad) [+ trunc_i(W^m_i, wd): weight decay, SVM R24]; W_i = trunc_i(W^m_i, s_fwd)
+// (R14, R21)
 template <typename T>
-__global__ void update_kernel(Pair<T> Wm, Pair<T> W, CPair<T> g, int64_t n, int s_grad, int s_fwd, int only = -1) {
+__global__ void update_kernel(Pair<T> Wm, Pair<T> W, CPair<T> g, int64_t n, int s_grad, int s_fwd, int only = -1,
+                              int wd = 0) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
 #pragma unroll
         for (int p = 0; p < 2; ++p) {
             if (only >= 0 && p != only) continue;
-            T wm = Wm.p[p][i] - trunc_share<T>(g.p[p][i], p, s_grad);
+            const T old = Wm.p[p][i];
+            const T dec = wd ? trunc_share<T>(old, p, wd) : (T)0;
+            T wm = old - (trunc_share<T>(g.p[p][i], p, s_grad) + dec);
             Wm.p[p][i] = wm;
             W.p[p][i] = trunc_share<T>(wm, p, s_fwd);
         }

@@ -205,7 +205,7 @@ static void add_msb(psml_model_s *m, int layer, int op, int64_t n, bool fwd) {
     m->items[0].push_back(it);
 }
 
-static bool is_eq9_out(const psml_model_s *m) { return m->d.kind != PSML_LINREG; }
+static bool is_eq9_out(const psml_model_s *m) { return m->d.kind != PSML_LINREG && m->d.kind != PSML_SVM; }
 // forward-weight fractional bits of layer l (R21)
 static int fw(const psml_model_s *m, int l) {
     const int v = m->d.fwd_frac_bits[l];
@@ -240,6 +240,14 @@ static void plan_items(psml_model_s *m) {
         cg.kind = IT_CONV_GW; cg.layer = 0; cg.op = OP_GRADW; cg.slot = 0;
         cg.M = kk; cg.K = rows; cg.N = m->cols[0]; cg.fwd = false;
         m->items[0].push_back(cg);
+        return;
+    }
+    if (m->d.kind == PSML_SVM) {   // linear SVM, hinge subgradient (R24)
+        add_matrix(m, 0, OP_FWD, B, m->dims[0], 1, true);
+        add_had(m, 0, 3, B, false);                 // margin y (.) z
+        add_msb(m, 0, OP_RELU_MSB, B, false);       // [y z - 1 < 0]
+        add_had(m, 0, 4, B, false);                 // y (.) ind
+        add_matrix(m, 0, OP_GRADW, m->dims[0], B, 1, false);
         return;
     }
     const int nl = m->nl;
@@ -669,6 +677,50 @@ static T *const *gradp(psml_model_s *m, int layer, T *tmp[2]) {
     return tmp;
 }
 
+// out_p = (neg ? -in_p : in_p) + [p == 0] c   (public constants are added by party 0)
+static __global__ void affine_pair_kernel(CPair<T> in, int64_t n, T c, int neg, Pair<T> out) {
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x)
+#pragma unroll
+        for (int p = 0; p < 2; ++p) {
+            const T v = neg ? (T)0 - in.p[p][e] : in.p[p][e];
+            out.p[p][e] = p == 0 ? v + c : v;
+        }
+}
+
+// Linear SVM (R24): m = trunc(y (.) z, F); ind = [m - 1 < 0]; delta = -(y (.) ind).
+static psml_status svm_delta(psml_model_s *m, const T *const z[2], const T *const Y[2], cudaStream_t s) {
+    const int F = m->ctx->ring.frac_bits;
+    const int64_t n = m->B;
+    DealItem *h3 = find_item(m, 0, OP_HADAMARD, 3), *h4 = find_item(m, 0, OP_HADAMARD, 4);
+    DealItem *cmp = find_item(m, 0, OP_RELU_MSB, 0);
+    if (!h3 || !h4 || !cmp) return fail(PSML_ERR_STATE, "missing SVM material");
+    T *mg[2] = {m->tmp.p[0], m->tmp.p[1]};                 // margin, then m - 1
+    T *ind[2] = {m->tmp.p[0] + n, m->tmp.p[1] + n};
+    T *c[2] = {m->tmp.p[0] + 2 * n, m->tmp.p[1] + 2 * n};
+    T *ws = m->ws;
+    PSML_TRY(beaver_hadamard<T>(Y, z, h3->U.cp(), h3->V.cp(), h3->Z.cp(), n, F, mg, ws, s));
+    affine_pair_kernel<<<ew_grid(n), EW_THREADS, 0, s>>>(CPair<T>{{mg[0], mg[1]}}, n, (T)0 - ((T)1 << F), 0,
+                                                         Pair<T>{{mg[0], mg[1]}});
+    PSML_LAUNCH_CHECK();
+    const T *t[2] = {mg[0], mg[1]};
+    if (cmp->kind == IT_FSS) {   // [t < 0] = 1 - DReLU(t)
+        PSML_TRY(fss_drelu_launch(CPair<T>{{t[0], t[1]}}, n, CPair<T>{{cmp->mat.p[0], cmp->mat.p[1]}},
+                                  Pair<T>{{ind[0], ind[1]}}, nullptr, ws, s));
+        affine_pair_kernel<<<ew_grid(n), EW_THREADS, 0, s>>>(CPair<T>{{ind[0], ind[1]}}, n, (T)1, 1,
+                                                             Pair<T>{{ind[0], ind[1]}});
+        PSML_LAUNCH_CHECK();
+    } else {                     // the A2B chain's arithmetic MSB shares
+        PSML_TRY(msb_chain<T>(t, n, cmp->mat.cp(), 0, 0, 0, ind, nullptr, nullptr, nullptr, nullptr, nullptr,
+                              nullptr, nullptr, nullptr, ws, s));
+    }
+    const T *ic[2] = {ind[0], ind[1]};
+    PSML_TRY(beaver_hadamard<T>(Y, ic, h4->U.cp(), h4->V.cp(), h4->Z.cp(), n, 0, c, ws, s));
+    affine_pair_kernel<<<ew_grid(n), EW_THREADS, 0, s>>>(CPair<T>{{c[0], c[1]}}, n, (T)0, 1,
+                                                         Pair<T>{{m->delta.p[0], m->delta.p[1]}});
+    PSML_LAUNCH_CHECK();
+    return PSML_OK;
+}
+
 // forward pass; if Y != nullptr also leaves delta = yhat - Y in m->delta
 static psml_status forward(psml_model_s *m, const T *const X[2], const T *const Y[2], T *const out[2],
                            cudaStream_t s) {
@@ -676,6 +728,13 @@ static psml_status forward(psml_model_s *m, const T *const X[2], const T *const 
     m->act[0].p[0] = (T *)X[0];
     m->act[0].p[1] = (T *)X[1];
     T *yo[2] = {out ? out[0] : m->yhat.p[0], out ? out[1] : m->yhat.p[1]};
+    if (m->d.kind == PSML_SVM) {
+        PSML_TRY(mm(m, m->act[0].cp(), m->W[0].cp(), 0, OP_FWD, 0, fw(m, 0), m->z[0].pp(), s));
+        const int64_t n = m->B;
+        for (int p = 0; p < 2; ++p)
+            PSML_CUDA_TRY(cudaMemcpyAsync(yo[p], m->z[0].p[p], sizeof(T) * n, cudaMemcpyDeviceToDevice, s));
+        return Y ? svm_delta(m, m->z[0].cp(), Y, s) : PSML_OK;
+    }
     if (m->d.kind == PSML_CNN) {
         PSML_TRY(conv(m, X, m->W[0].cp(), 0, fw(m, 0), m->z[0].pp(), s));
         PSML_TRY(relu(m, m->z[0].cp(), 0, m->act[1].pp(), m->drelu[0].pp(), s));
@@ -704,6 +763,8 @@ static psml_status forward(psml_model_s *m, const T *const X[2], const T *const 
 static psml_status backward(psml_model_s *m, cudaStream_t s) {
     const int F = m->ctx->ring.frac_bits;
     T *g[2];
+    if (m->d.kind == PSML_SVM)
+        return mm(m, m->act[0].cp(), m->delta.cp(), 0, OP_GRADW, PSML_TRANS_A, 0, gradp(m, 0, g), s);
     if (m->d.kind == PSML_CNN) {
         // layer 2 (FC 64 -> 10)
         PSML_TRY(mm(m, m->act[2].cp(), m->delta.cp(), 2, OP_GRADW, PSML_TRANS_A, 0, gradp(m, 2, g), s));
@@ -739,7 +800,9 @@ static int item_index(const psml_model_s *m, int layer, int op, int slot) {
 }
 
 static bool fused_eligible(const psml_model_s *m) {
-    if (m->d.kind == PSML_CNN || m->nl > UPD_MAX_LAYERS || (int)m->ob.size() != (int)m->items[0].size()) return false;
+    if (m->d.kind == PSML_CNN || m->d.kind == PSML_SVM || m->nl > UPD_MAX_LAYERS ||
+        (int)m->ob.size() != (int)m->items[0].size())
+        return false;
     for (int l = 0; l < m->nl; ++l)
         if (fw(m, l) != m->ctx->ring.frac_bits) return false;   // the fused step truncates by F
     if (m->d.compare != 0) return false;                         // the fused step runs the A2B chain
@@ -1276,9 +1339,11 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
     switch (desc->kind) {
     case PSML_LINREG:
     case PSML_LOGREG:
+    case PSML_SVM:
     case PSML_MLP: {
         int nl = desc->n_layers;
         if (desc->kind != PSML_MLP) nl = 1;
+        if (desc->kind == PSML_SVM && desc->dims[1] != 1) return fail(PSML_ERR_SHAPE, "SVM: dims = {d, 1}");
         if (nl < 1 || nl > 7) return fail(PSML_ERR_SHAPE, "n_layers must be in [1, 7]");
         for (int i = 0; i <= nl; ++i)
             if (desc->dims[i] <= 0) return fail(PSML_ERR_SHAPE, "dims must be positive");
@@ -1306,6 +1371,8 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
     default:
         return fail(PSML_ERR_INVALID, "unknown model kind");
     }
+    if (desc->weight_decay_shift < 0 || desc->weight_decay_shift >= 64)
+        return fail(PSML_ERR_INVALID, "weight_decay_shift must be in [0, 64)");
     for (int l = 0; l < m->nl; ++l) {
         const int v = desc->fwd_frac_bits[l];
         if (v != 0 && (v < c->ring.frac_bits || v > desc->master_frac_bits))
@@ -1338,7 +1405,7 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
     }
     PSML_TRY(balloc(mp, m->yhat, B * m->dims[m->nl]));
     PSML_TRY(balloc(mp, m->delta, B * maxw));
-    PSML_TRY(balloc(mp, m->tmp, B * maxw));
+    PSML_TRY(balloc(mp, m->tmp, B * std::max<int64_t>(maxw, 3)));   // SVM: margin, indicator, y (.) ind
     if (m->d.kind == PSML_CNN) {   // im2col column offsets (ch, ky, kx) -> ch*H*W + ky*W + kx
         const ConvGeom &g = m->g;
         std::vector<int32_t> off((size_t)g.C * g.k * g.k);
@@ -1505,7 +1572,7 @@ psml_status psml_train_apply_update(psml_model m, int32_t extra_shift, psml_stre
             tot += m->rows[l] * m->cols[l];
         }
         u.begin[m->nl] = tot;
-        u.nl = m->nl; u.s_grad = s_grad;
+        u.nl = m->nl; u.s_grad = s_grad; u.wd = m->d.weight_decay_shift;
         for (int l = 0; l < m->nl; ++l) u.s_fwd[l] = m->d.master_frac_bits - fw(m, l);
         PSML_CUDA_TRY(launch_pdl(update_all_kernel<T>, dim3(ew_grid(tot)), dim3(EW_THREADS), s, u));
         PSML_LAUNCH_CHECK();
@@ -1519,7 +1586,8 @@ psml_status psml_train_apply_update(psml_model m, int32_t extra_shift, psml_stre
         update_kernel<T><<<ew_grid(n), EW_THREADS, 0, s>>>(Pair<T>{{m->Wm[l].p[0], m->Wm[l].p[1]}},
                                                             Pair<T>{{m->W[l].p[0], m->W[l].p[1]}},
                                                             CPair<T>{{g[0], g[1]}}, n, s_grad,
-                                                            m->d.master_frac_bits - fw(m, l));
+                                                            m->d.master_frac_bits - fw(m, l), -1,
+                                                            m->d.weight_decay_shift);
         PSML_LAUNCH_CHECK();
     }
     m->grads_ready = false;
@@ -1869,6 +1937,7 @@ psml_status psml_party_forward_backward(psml_model m, int32_t party, psml_xport 
                                         uint32_t step_id, psml_stream stream) {
     if (!m || !x) return fail(PSML_ERR_INVALID, "null model or transport");
     if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
+    if (m->d.kind == PSML_SVM) return fail(PSML_ERR_UNSUPPORTED, "SVM: co-resident engine only");
     PSML_TRY(check_ptrs({X_i, Y_i}));
     const int pool = (int)(step_id & 1);
     if (m->dealt_step[pool] != (int64_t)step_id || !m->dealt_full[pool])
@@ -1903,7 +1972,8 @@ psml_status psml_party_apply_update(psml_model m, int32_t party, int32_t extra_s
         update_kernel<T><<<ew_grid(n), EW_THREADS, 0, s>>>(Pair<T>{{m->Wm[l].p[0], m->Wm[l].p[1]}},
                                                             Pair<T>{{m->W[l].p[0], m->W[l].p[1]}},
                                                             CPair<T>{{g[0], g[1]}}, n, s_grad,
-                                                            m->d.master_frac_bits - fw(m, l), party);
+                                                            m->d.master_frac_bits - fw(m, l), party,
+                                                            m->d.weight_decay_shift);
         PSML_LAUNCH_CHECK();
     }
     m->grads_ready = false;

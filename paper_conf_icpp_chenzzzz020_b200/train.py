@@ -23,7 +23,8 @@ SHARE_SEED = DATA_SEED + 1
 DEALER_SEED = DATA_SEED + 2
 OP_SHARE = 7
 INIT_STEP = 0xFFFFFFFF
-KINDS = {"linreg": psml.LINREG, "logreg": psml.LOGREG, "mlp": psml.MLP, "cnn": psml.CNN}
+KINDS = {"linreg": psml.LINREG, "logreg": psml.LOGREG, "mlp": psml.MLP, "cnn": psml.CNN, "svm": psml.SVM}
+WD_SHIFT = {"svm": 16}   # weight decay lambda.eta = 2^-16 (R24)
 # forward-weight fractional bits per layer (R21); None = frac_bits for every layer
 FWD_BITS = {"cnn": [16, 20, 20]}
 
@@ -47,7 +48,7 @@ class SecureTrainer:
         self.model = psml.Model(self.ctx, KINDS[task], dims=dims, batch=batch, lr_shift=lr_shift,
                                 master_frac_bits=master_frac_bits, dealer_seed=DEALER_SEED,
                                 pair_id=pair_id, fwd_frac_bits=FWD_BITS.get(task),
-                                compare={"a2b": 0, "fss": 1}[compare])
+                                compare={"a2b": 0, "fss": 1}[compare], weight_decay_shift=WD_SHIFT.get(task, 0))
         for layer, W in enumerate(W_init):
             w = psml.encode(self.master_ring, torch.as_tensor(W, dtype=torch.float64))
             Wm = psml.share(self.ring, SHARE_SEED, call_id(0, INIT_STEP, layer, OP_SHARE, 2), w)

@@ -112,6 +112,8 @@ def labels(task, X):
         return X @ linear_teacher()
     if task == "logreg":
         return (X @ linear_teacher() > logistic_threshold()).astype(np.float64)
+    if task == "svm":      # +-1 labels of the same linear teacher (R24)
+        return np.where(X @ linear_teacher() > logistic_threshold(), 1.0, -1.0)
     if task == "mlp":
         W = mlp_teacher()
         return _one_hot(relu(relu(X @ W[0]) @ W[1]) @ W[2])
@@ -122,7 +124,7 @@ def labels(task, X):
     raise ValueError(task)
 
 
-TASK_DATA = {"linreg": "mnist", "logreg": "mnist", "mlp": "mnist", "cnn": "cifar"}
+TASK_DATA = {"linreg": "mnist", "logreg": "mnist", "svm": "mnist", "mlp": "mnist", "cnn": "cifar"}
 TASK_ROWS = {"mnist": 60000, "cifar": 50000}
 
 
@@ -151,7 +153,7 @@ def batch_u8(task, step, batch_size=BLOCK, pair=0, n_pairs=1, seed=DATA_SEED):
 def init_weights(task, dims=None, seed=INIT_SEED):
     """Initial plaintext weights (R13): zeros for linear/logistic regression,
     U(+-1/sqrt(fan_in)) for the MLP and CNN."""
-    if task in ("linreg", "logreg"):
+    if task in ("linreg", "logreg", "svm"):
         return [np.zeros((MNIST_FEATURES, 1))]
     if task == "mlp":
         dims = dims or (784, 128, 128, 10)

@@ -297,3 +297,34 @@ def test_forward_weight_precision_bookkeeping(orc, fw):
     got = orc.decode(orc.reconstruct(*z), 64, P.F)
     want = plain.q(Xf, P.F) @ Wf
     assert np.abs(got - want).max() < 40 * 2.0 ** -fw + 2 * 2.0 ** -P.F
+
+
+@pytest.mark.parametrize("compare", ["a2b", "fss"])
+def test_svm_training_tracks_fp64(compare):
+    """Linear SVM (R24): hinge-loss subgradient + weight decay; decoded master weights
+    vs fp64 with the same rule, zero comparison mismatches / truncation failures."""
+    task = "svm"
+    Wi = synth.init_weights(task)
+    m, pm = P.Model(task, Wi, compare=compare), plain.PlainModel(task, Wi)
+    P.diag_reset(True)
+    try:
+        for s in range(30):
+            X, Y = synth.batch(task, s)
+            P.train_step(m, X, Y, s)
+            pm.step(X, Y)
+        d = dict(P.DIAG)
+    finally:
+        P.diag_reset(False)
+    assert d["msb_fail"] == 0 and d["trunc_fail"] == 0 and d["msb_checked"] == 30 * 128, d
+    err = np.abs(m.decoded_master()[0] - pm.W[0]).max()
+    assert err < 2.0 ** -16, np.log2(err)
+
+
+@pytest.mark.parametrize("compare", ["a2b", "fss"])
+def test_comparison_lt0_edges(orc, compare):
+    """[t < 0] shares (the SVM's hinge indicator) on l = 64 edge values, both comparisons."""
+    edges = [0, 1, (1 << 63) - 1, 1 << 63, (1 << 64) - 1, 1 << 13, (1 << 64) - (1 << 13)]
+    t = np.array(edges * 20, dtype=np.uint64)
+    t0 = orc.prg(64, 21, orc.tag("tt"), 0, t.size)
+    got = P.comparison_lt0((t0, t - t0), 0, 9, 0, compare)
+    assert np.array_equal(got[0] + got[1], (t.view(np.int64) < 0).astype(np.uint64))
