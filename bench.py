@@ -507,8 +507,8 @@ PROF_CLASS = {0: "ring_gemm_cuda_core", 1: "ring_gemm_tcgen05", 2: "msb_relu_eq9
 # kernel name -> class (CUPTI records); the dealer's Z = U V products are dealer work
 KERNEL_CLASS = (("ring_gemm_cl_grouped", "dealer"), ("deal_prg", "dealer"), ("dealer_", "dealer"),
                 ("hadamard_triplet", "dealer"), ("msb_dealer", "dealer"), ("prg_kernel", "dealer"),
-                ("seg_gemm", "ring_gemm_cuda_core"), ("ring_gemm", "ring_gemm_cuda_core"),
                 ("tc_seg", "ring_gemm_tcgen05"), ("tc_ring", "ring_gemm_tcgen05"),
+                ("seg_gemm", "ring_gemm_cuda_core"), ("ring_gemm", "ring_gemm_cuda_core"),
                 ("msb_", "msb_relu_eq9_rounds"), ("had_", "hadamard_rounds"), ("hadamard", "hadamard_rounds"),
                 ("eq9", "hadamard_rounds"), ("open", "beaver_mask"), ("mask", "beaver_mask"),
                 ("update", "update"), ("encode_share", "client_share"), ("client_share", "client_share"))

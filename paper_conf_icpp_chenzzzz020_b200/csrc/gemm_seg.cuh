@@ -249,15 +249,11 @@ bool tc_seg_enabled();
 bool tc_seg_forced();   // PSML_SEG=tc: every eligible group on tcgen05 (tests)
 bool pdl_enabled();     // PSML_PDL=0 disables programmatic dependent launch
 psml_status tc_seg_group(const SegArgs<uint64_t> *jobs, int njobs, cudaStream_t stream, int sm_count);
-size_t tc_limb_seg_ws_bytes(int64_t M, int64_t K, int64_t N);
-psml_status tc_limb_seg_group(const SegArgs<uint64_t> *jobs, int njobs, void *ws, size_t ws_bytes, cudaStream_t s,
-                              int sm_count);
-int tc_seg_route();   // PSML_TCSEG: 0 = in-kernel split (tc_seg_kernel), 1 = limb planes + v4
+
 
 // Launch 1..SEG_MAX_JOBS products as one grid; the cluster split ks is chosen for the group.
 template <typename T>
-psml_status launch_seg_group(const SegArgs<T> *jobs, int njobs, cudaStream_t stream, int sm_count,
-                             void *tcws = nullptr, size_t tcws_bytes = 0) {
+psml_status launch_seg_group(const SegArgs<T> *jobs, int njobs, cudaStream_t stream, int sm_count) {
     using C = SegCfg;
     if (njobs < 1 || njobs > SEG_MAX_JOBS) return fail(PSML_ERR_INVALID, "seg group: 1..4 jobs");
     if constexpr (sizeof(T) == 8) {
@@ -270,12 +266,8 @@ psml_status launch_seg_group(const SegArgs<T> *jobs, int njobs, cudaStream_t str
             ok = 2 * jobs[q].K <= 16384;
             macs += (double)jobs[q].M * jobs[q].N * 2 * jobs[q].K * jobs[q].nparty;
         }
-        if (ok && (macs >= (double)(1 << 25) || tc_seg_forced())) {
-            if (tc_seg_route() == 1 && tcws)
-                return tc_limb_seg_group(reinterpret_cast<const SegArgs<uint64_t> *>(jobs), njobs, tcws, tcws_bytes,
-                                         stream, sm_count);
+        if (ok && (macs >= (double)(1 << 25) || tc_seg_forced()))
             return tc_seg_group(reinterpret_cast<const SegArgs<uint64_t> *>(jobs), njobs, stream, sm_count);
-        }
     }
     SegGroup<T> g{};
     int64_t tiles = 0, kmax = 0;

@@ -593,14 +593,14 @@ static psml_status launch_split(const SplitJobs &jobs, cudaStream_t s) {
 // Picks split-K (fills the SMs, keeps each l = 64 pass exact) and launches GEMM (+ finalize).
 template <int l>
 static psml_status launch_gemm(TcParams<typename Cfg<l>::T> P, int64_t Mp, int64_t Np, typename Cfg<l>::T *partial,
-                               int64_t partial_words, int sm_count, cudaStream_t s, int min_kb_per_split = 8) {
+                               int64_t partial_words, int sm_count, cudaStream_t s) {
     using T = typename Cfg<l>::T;
     constexpr int BN = Cfg<l>::BN;
     const int nkb = P.nkb_lo + P.nkb_hi;
     const int64_t tiles = (Mp / BM) * (Np / BN) * P.nparty;   // CTAs per split (pairs count 2)
     int splits = 1;
     if (tiles < sm_count)
-        splits = (int)std::min<int64_t>((sm_count + tiles - 1) / tiles, std::max(1, nkb / min_kb_per_split));
+        splits = (int)std::min<int64_t>((sm_count + tiles - 1) / tiles, std::max(1, nkb / 8));
     splits = std::max(splits, (nkb + Cfg<l>::MAX_KB - 1) / Cfg<l>::MAX_KB);
     int kbs = (nkb + splits - 1) / splits;
     splits = (nkb + kbs - 1) / kbs;
@@ -834,60 +834,5 @@ template psml_status tc_beaver_matmul<uint32_t>(Ctx *, const uint32_t *const[2],
                                                 const uint32_t *const[2], const uint32_t *const[2],
                                                 const uint32_t *const[2], int64_t, int64_t, int64_t, int, int,
                                                 uint32_t *const[2], cudaStream_t);
-
-// ------------------------------------------------------------------------------------------------
-// The training step's two-segment Beaver products on tcgen05 from limb planes (co-resident engine):
-// C_p = [X_p | E] . [F ; V_p] + Z_p, truncated (gemm_seg.cuh SegArgs).  One split pass writes the
-// limb planes of X_0, X_1, E (A operands) and F, V_0, V_1 (B operands) into the UMMA canonical
-// layout, then tc_ring_gemm64_v4 runs the 36 limb-pair MMAs per K block with split-K over (nearly)
-// every SM -- the MLP's products are one 128 x 128 tile per party -- and the finalize pass adds Z_p
-// and truncates.  ws: tc_limb_seg_ws_bytes(M, K, N) bytes per job.
-// ------------------------------------------------------------------------------------------------
-size_t tc_limb_seg_ws_bytes(int64_t M, int64_t K, int64_t N) {
-    const int64_t ta = tc::tiled_bytes<64>(M, K, tc::BM), tb = tc::tiled_bytes<64>(N, K, tc::Cfg<64>::BN);
-    return (size_t)(3 * ((ta + 255) & ~255) + 3 * ((tb + 255) & ~255) + 2 * 8 * M * N + 4096);
-}
-
-psml_status tc_limb_seg_group(const SegArgs<uint64_t> *jobs, int njobs, void *ws, size_t ws_bytes,
-                              cudaStream_t s, int sm_count) {
-    using Cf = tc::Cfg<64>;
-    using T = uint64_t;
-    uint8_t *w = (uint8_t *)ws;
-    size_t used = 0;
-    for (int q = 0; q < njobs; ++q) {
-        const SegArgs<T> &a = jobs[q];
-        if (a.nparty != 2) return fail(PSML_ERR_UNSUPPORTED, "limb-plane seg GEMM: co-resident pairs only");
-        const size_t need = tc_limb_seg_ws_bytes(a.M, a.K, a.N);
-        if (!ws || used + need > ws_bytes) return fail(PSML_ERR_NOMEM, "limb-plane seg GEMM workspace too small");
-        const int64_t ta = tc::tiled_bytes<64>(a.M, a.K, tc::BM), tb = tc::tiled_bytes<64>(a.N, a.K, Cf::BN);
-        uint8_t *base = w + used;
-        auto carve = [&](size_t bytes) { uint8_t *p = base; base += (bytes + 255) & ~(size_t)255; return p; };
-        uint8_t *tX0 = carve(ta), *tX1 = carve(ta), *tE = carve(ta), *tF = carve(tb), *tV0 = carve(tb), *tV1 = carve(tb);
-        T *partial = (T *)carve(sizeof(T) * 2 * a.M * a.N);
-        used += need;
-        tc::SplitJobs sj;
-        sj.j[0] = tc::make_job<64>(a.X[0], nullptr, nullptr, tX0, a.M, a.K, tc::BM, 0);
-        sj.j[1] = tc::make_job<64>(a.X[1], nullptr, nullptr, tX1, a.M, a.K, tc::BM, 0);
-        sj.j[2] = tc::make_job<64>(a.E, nullptr, nullptr, tE, a.M, a.K, tc::BM, 0);
-        sj.j[3] = tc::make_job<64>(a.F, nullptr, nullptr, tF, a.N, a.K, Cf::BN, 1);
-        sj.j[4] = tc::make_job<64>(a.V[0], nullptr, nullptr, tV0, a.N, a.K, Cf::BN, 1);
-        sj.j[5] = tc::make_job<64>(a.V[1], nullptr, nullptr, tV1, a.N, a.K, Cf::BN, 1);
-        sj.count = 6;
-        {
-            ProfScope prof(PROF_TC, s, 0.0);
-            PSML_TRY(tc::launch_split<64>(sj, s));
-        }
-        tc::TcParams<T> P{};
-        P.A_lo[0] = tX0; P.A_lo[1] = tX1; P.A_hi[0] = P.A_hi[1] = tE;
-        P.B_lo[0] = P.B_lo[1] = tF; P.B_hi[0] = tV0; P.B_hi[1] = tV1;
-        P.a_stride_lo = P.a_stride_hi = sj.j[0].rows_pad * sj.j[0].k_pad;
-        P.b_stride_lo = P.b_stride_hi = sj.j[3].rows_pad * sj.j[3].k_pad;
-        P.nkb_lo = P.nkb_hi = (int)(sj.j[0].k_pad / tc::BK);
-        P.M = a.M; P.N = a.N; P.nparty = 2; P.mode = 1; P.trunc = a.trunc;
-        for (int p = 0; p < 2; ++p) { P.C[p] = a.C[p]; P.Z[p] = a.Z[p]; }
-        PSML_TRY(tc::launch_gemm<64>(P, sj.j[0].rows_pad, sj.j[3].rows_pad, partial, 2 * a.M * a.N, sm_count, s, 2));
-    }
-    return PSML_OK;
-}
 
 }  // namespace psml

@@ -443,15 +443,6 @@ __global__ void __launch_bounds__(NT, 1) tc_seg_kernel(const __grid_constant__ G
 
 }  // namespace tcseg
 
-int tc_seg_route() {
-    static int v = -1;
-    if (v < 0) {
-        const char *e = getenv("PSML_TCSEG");
-        v = (e && e[0] == '1') ? 1 : 0;
-    }
-    return v;
-}
-
 bool tc_seg_forced() {
     static int v = -1;
     if (v < 0) {

@@ -156,8 +156,6 @@ struct psml_model_s {
     // split deployment capture (psml_party_capture_step): the party, its pair transport and its
     // data-parallel communicator; cap_party < 0 = the co-resident engine
     int cap_party = -1;
-    void *tcws = nullptr;              // limb planes of the tcgen05-sized products (tc_limb_seg_group)
-    size_t tcws_bytes = 0;
     psml_xport cap_xport = nullptr;
     psml_dp cap_dp = nullptr;
 };
@@ -818,20 +816,12 @@ static bool fused_shapes_ok(const psml_model_s *m) {
 
 static psml_status alloc_open_bufs(psml_model_s *m) {
     m->ob.assign(m->items[0].size(), OpenBuf{});
-    size_t tcb = 0;
     for (size_t k = 0; k < m->items[0].size(); ++k) {
         const DealItem &it = m->items[0][k];
         if (it.kind != IT_MATRIX) continue;
         PSML_TRY(dalloc(m, &m->ob[k].E, it.M * it.K));
         PSML_TRY(dalloc(m, &m->ob[k].X1, it.M * it.K));
         PSML_TRY(dalloc(m, &m->ob[k].F, it.K * it.N));
-        if ((double)it.M * it.N * 2 * it.K * 2 >= (double)(1 << 25)) tcb += tc_limb_seg_ws_bytes(it.M, it.K, it.N);
-    }
-    if (tcb) {
-        T *p = nullptr;
-        PSML_TRY(dalloc(m, &p, (int64_t)(tcb / sizeof(T)) + 1));
-        m->tcws = p;
-        m->tcws_bytes = tcb;
     }
     return PSML_OK;
 }
@@ -943,7 +933,7 @@ static psml_status fused_forward_backward(psml_model_s *m, const T *const X[2], 
     T *yo[2] = {m->yhat.p[0], m->yhat.p[1]};
     for (int l = 0; l < nl; ++l) {
         SegArgs<T> a = seg(l, OP_FWD, m->z[l].p[0], m->z[l].p[1], F);
-        PSML_TRY(launch_seg_group<T>(&a, 1, s, m->ctx->sm_count, m->tcws, m->tcws_bytes));
+        PSML_TRY(launch_seg_group<T>(&a, 1, s, m->ctx->sm_count));
         PSML_TRY(deal_fork_point(m, s));
         const int64_t w = m->dims[l + 1];
         if (l < nl - 1) {
@@ -995,10 +985,10 @@ static psml_status fused_forward_backward(psml_model_s *m, const T *const X[2], 
         if (branch && l > 0) {
             PSML_CUDA_TRY(cudaEventRecord(m->ev_gw, s));
             PSML_CUDA_TRY(cudaStreamWaitEvent(m->gw, m->ev_gw, 0));
-            PSML_TRY(launch_seg_group<T>(&jobs[0], 1, m->gw, m->ctx->sm_count, m->tcws, m->tcws_bytes));
-            PSML_TRY(launch_seg_group<T>(&jobs[1], 1, s, m->ctx->sm_count, m->tcws, m->tcws_bytes));
+            PSML_TRY(launch_seg_group<T>(&jobs[0], 1, m->gw, m->ctx->sm_count));
+            PSML_TRY(launch_seg_group<T>(&jobs[1], 1, s, m->ctx->sm_count));
         } else {
-            PSML_TRY(launch_seg_group<T>(jobs, l > 0 ? 2 : 1, s, m->ctx->sm_count, m->tcws, m->tcws_bytes));
+            PSML_TRY(launch_seg_group<T>(jobs, l > 0 ? 2 : 1, s, m->ctx->sm_count));
         }
         PSML_TRY(deal_fork_point(m, s));
         if (l > 0) {
