@@ -281,7 +281,11 @@ psml_status psml_delta_apply(psml_ctx ctx, int64_t rows, int64_t cols, int32_t i
  * SVM trained by SMO; R24 reads it as the primal subgradient form that runs on the
  * Beaver / comparison primitives): z = X w; ind = [y z < 1]; gradW = X^T (-(y (.) ind)); labels
  * +-1.  Co-resident engine only. */
-typedef enum { PSML_LINREG = 0, PSML_LOGREG = 1, PSML_MLP = 2, PSML_CNN = 3, PSML_SVM = 4 } psml_model_kind;
+/* PSML_RNN: Elman RNN over rnn_steps = T steps (R25): dims = {D, H, C},
+ * X: batch x (T D) (step t = columns t D .. (t+1) D), h_t = ReLU([x_t | h_{t-1}] . W_1) with W_1 of
+ * (D + H) x H, yhat = Eq9(h_T . W_o) with W_o of H x C; trained by backpropagation through time
+ * (the weight gradient of W_1 is the ring sum over t).  Co-resident engine only. */
+typedef enum { PSML_LINREG = 0, PSML_LOGREG = 1, PSML_MLP = 2, PSML_CNN = 3, PSML_SVM = 4, PSML_RNN = 5 } psml_model_kind;
 
 typedef struct {
     int32_t kind;             /* psml_model_kind                                             */
@@ -301,6 +305,7 @@ typedef struct {
                                  DCF comparison (R22; material psml_fss_dealer's layout)       */
     int32_t weight_decay_shift; /* 0 = none; else W^m -= trunc(W^m, shift) every update (SVM:
                                    lambda.eta = 2^-16, R24)                        */
+    int32_t rnn_steps;        /* RNN: sequence length T (1..254; call-id layers 1..T+1)       */
 } psml_model_desc;
 
 psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_model *out);

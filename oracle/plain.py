@@ -12,7 +12,7 @@ only differences from the secure run are fixed-point rounding and truncation noi
 """
 import numpy as np
 
-from .protocol import F, LR_SHIFT, MASTER, CNN_GEOM, WD_SHIFT
+from .protocol import F, LR_SHIFT, MASTER, CNN_GEOM, WD_SHIFT, RNN_GEOM
 
 
 def q(x, f):
@@ -82,6 +82,8 @@ class PlainModel:
 
     def step(self, X, Y):
         X, Y = q(X, F), q(Y, F)
+        if self.task == "rnn":   # backpropagation through time (R25)
+            return self._rnn_step(X, Y)
         acts, masks, yhat = self.forward(X)
         if self.task == "svm":   # hinge subgradient + weight decay (R24)
             delta = -Y * ((Y * yhat) < 1.0)
@@ -103,4 +105,29 @@ class PlainModel:
                 delta = (delta @ self.W[layer].T) * masks[layer - 1]
         for layer, gr in enumerate(grads):
             self.W[layer] = self.W[layer] - lr * gr
+        return yhat
+
+    def _rnn_step(self, X, Y):
+        g = RNN_GEOM
+        T, D, H = g["T"], g["D"], g["H"]
+        W1, Wo = self.W
+        h = np.zeros((X.shape[0], H))
+        As, masks = [], []
+        for t in range(T):
+            A = np.concatenate([X[:, t * D:(t + 1) * D], h], axis=1)
+            z = A @ W1
+            As.append(A)
+            masks.append(z >= 0)
+            h = np.maximum(z, 0.0)
+        yhat = eq9(h @ Wo)
+        delta = yhat - Y
+        gWo = h.T @ delta
+        delta = (delta @ Wo.T) * masks[T - 1]
+        gW1 = np.zeros_like(W1)
+        for t in range(T - 1, -1, -1):
+            gW1 += As[t].T @ delta
+            if t > 0:
+                delta = (delta @ W1[D:, :].T) * masks[t - 1]
+        lr = 2.0 ** -LR_SHIFT
+        self.W = [W1 - lr * gW1, Wo - lr * gWo]
         return yhat

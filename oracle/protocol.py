@@ -37,7 +37,8 @@ CNN_GEOM = dict(C=3, H=32, W=32, k=5, Cout=16, hidden=64, classes=10)
 # h.W and backprop delta.W^T) is truncated by f_w, so activations and deltas stay at F = 13 bits.
 # f_w = F except the CNN, whose 12544-wide FC1 and 5x5 conv fail BJ's 2^-12 weight bound at
 # f_w = 13 (weights of magnitude ~0.005 quantised at 2^-13 perturb every pre-activation).
-FWD_BITS = {"linreg": [F], "logreg": [F], "svm": [F], "mlp": [F, F, F], "cnn": [16, 20, 20]}
+FWD_BITS = {"linreg": [F], "logreg": [F], "svm": [F], "mlp": [F, F, F], "cnn": [16, 20, 20], "rnn": [F, F]}
+RNN_GEOM = dict(T=16, D=32, H=64, C=10)   # DESIGN.md R25 (synth.RNN_*)
 # linear SVM (R24): weight decay lambda.eta = 2^-WD_SHIFT applied to the master weights
 WD_SHIFT = 16
 
@@ -258,6 +259,48 @@ def _svm_forward_backward(model, Xs, Ys, step, pair):
     return grads, z
 
 
+def _rnn_forward(model, Xs, step, pair):
+    """Elman RNN (R25; "passes the states in its own network"):
+    h_0 = 0;  A_t = [x_t | h_{t-1}];  z_t = trunc(A_t . W_1, f_w);  h_t = ReLU(z_t)  (t = 1..T,
+    call-id layer t);  yhat = Eq9(trunc(h_T . W_o, f_w))  (layer T + 1)."""
+    g = RNN_GEOM
+    T, D, H = g["T"], g["D"], g["H"]
+    B = Xs[0].shape[0]
+    h = (np.zeros((B, H), np.uint64), np.zeros((B, H), np.uint64))
+    As, drelus = [], []
+    for t in range(1, T + 1):
+        A = tuple(np.ascontiguousarray(np.concatenate([x[:, (t - 1) * D:t * D], hh], axis=1)) for x, hh in zip(Xs, h))
+        z = matmul(A, model.W[0], pair, step, t, OP_FWD, model.fw[0])
+        h, d = relu(z, pair, step, t, model.compare)
+        As.append(A)
+        drelus.append(d)
+    zo = matmul(h, model.W[1], pair, step, T + 1, OP_FWD, model.fw[1])
+    return As, drelus, h, zo
+
+
+def _rnn_forward_backward(model, Xs, Ys, step, pair):
+    """Backpropagation through time: gW_o = h_T^T delta; delta_T = trunc(delta . W_o^T) (.) DReLU_T;
+    gW_1 = sum_t A_t^T delta_t (untruncated, ring addition); delta_{t-1} = trunc(delta_t . W_h^T)
+    (.) DReLU_{t-1} with W_h = the last H rows of W_1."""
+    g = RNN_GEOM
+    T, D = g["T"], g["D"]
+    As, drelus, h, zo = _rnn_forward(model, Xs, step, pair)
+    yhat = eq9(zo, pair, step, T + 1, model.compare)
+    delta = sub_pair(yhat, Ys)
+    gWo = matmul(_T(h), delta, pair, step, T + 1, OP_GRADW, 0)
+    t_ = matmul(delta, _T(model.W[1]), pair, step, T + 1, OP_GRADIN, model.fw[1])
+    delta = hadamard(t_, drelus[T - 1], pair, step, T, 1)
+    gW1 = (np.zeros(model.W[0][0].shape, np.uint64), np.zeros(model.W[0][0].shape, np.uint64))
+    for t in range(T, 0, -1):
+        gt = matmul(_T(As[t - 1]), delta, pair, step, t, OP_GRADW, 0)
+        gW1 = (gW1[0] + gt[0], gW1[1] + gt[1])
+        if t > 1:
+            Wh = tuple(np.ascontiguousarray(w[D:, :]) for w in model.W[0])
+            t_ = matmul(delta, _T(Wh), pair, step, t, OP_GRADIN, model.fw[0])
+            delta = hadamard(t_, drelus[t - 2], pair, step, t - 1, 1)
+    return [gW1, gWo], yhat
+
+
 def forward_backward(model, Xs, Ys, step, pair=0):
     """Returns (per-layer untruncated weight-gradient shares, prediction shares)."""
     task = model.task
@@ -265,6 +308,8 @@ def forward_backward(model, Xs, Ys, step, pair=0):
         return _cnn_forward_backward(model, Xs, Ys, step, pair)
     if task == "svm":
         return _svm_forward_backward(model, Xs, Ys, step, pair)
+    if task == "rnn":
+        return _rnn_forward_backward(model, Xs, Ys, step, pair)
     nl = len(model.W)
     acts = [Xs]
     drelus = []
@@ -342,6 +387,9 @@ def train_step(model, X, Y, step, pair=0):
 def infer(model, Xs, step, pair=0):
     """Secure inference = the forward half."""
     task = model.task
+    if task == "rnn":
+        _, _, _, zo = _rnn_forward(model, Xs, step, pair)
+        return eq9(zo, pair, step, RNN_GEOM["T"] + 1, model.compare)
     if task == "cnn":
         B = Xs[0].shape[0]
         U, V, Z = conv_triplet(pair, step, OP_FWD, B, transpose=False)

@@ -156,6 +156,10 @@ struct psml_model_s {
     // split deployment capture (psml_party_capture_step): the party, its pair transport and its
     // data-parallel communicator; cap_party < 0 = the co-resident engine
     int cap_party = -1;
+    // RNN (R25): per time step inputs A_t = [x_t | h_{t-1}], states h_t, DReLU_t, and the
+    // per-step weight-gradient product before it is added into the layer-0 gradient
+    psml::Buf rnnA, rnnH, rnnD, rnnG;
+    int rnn_T = 0, rnn_D = 0;
     psml_xport cap_xport = nullptr;
     psml_dp cap_dp = nullptr;
 };
@@ -238,6 +242,29 @@ static void plan_items(psml_model_s *m) {
         cg.kind = IT_CONV_GW; cg.layer = 0; cg.op = OP_GRADW; cg.slot = 0;
         cg.M = kk; cg.K = rows; cg.N = m->cols[0]; cg.fwd = false;
         m->items[0].push_back(cg);
+        return;
+    }
+    if (m->d.kind == PSML_RNN) {   // Elman RNN, backpropagation through time (R25)
+        const int T = m->rnn_T;
+        const int64_t K1 = m->rows[0], H = m->dims[1], C = m->dims[2];
+        for (int t = 1; t <= T; ++t) {
+            add_matrix(m, t, OP_FWD, B, K1, H, true);
+            add_msb(m, t, OP_RELU_MSB, B * H, true);
+            add_had(m, t, 0, B * H, true);
+        }
+        add_matrix(m, T + 1, OP_FWD, B, H, C, true);
+        add_msb(m, T + 1, OP_EQ9_MSB, 2 * B * C, true);
+        add_had(m, T + 1, 2, 2 * B * C, true);
+        add_matrix(m, T + 1, OP_GRADW, H, B, C, false);
+        add_matrix(m, T + 1, OP_GRADIN, B, C, H, false);
+        add_had(m, T, 1, B * H, false);
+        for (int t = T; t >= 1; --t) {
+            add_matrix(m, t, OP_GRADW, K1, B, H, false);
+            if (t > 1) {
+                add_matrix(m, t, OP_GRADIN, B, H, H, false);
+                add_had(m, t - 1, 1, B * H, false);
+            }
+        }
         return;
     }
     if (m->d.kind == PSML_SVM) {   // linear SVM, hinge subgradient (R24)
@@ -675,6 +702,24 @@ static T *const *gradp(psml_model_s *m, int layer, T *tmp[2]) {
     return tmp;
 }
 
+using T_ = T;
+// RNN input of step t: A[b, 0:D] = X[b, t D : (t + 1) D], A[b, D:D+H] = h_prev[b, :] (0 at t = 0)
+static __global__ void rnn_concat_kernel(CPair<T> X, CPair<T> hprev, int64_t B, int64_t D, int64_t H, int64_t xw, int t,
+                                         Pair<T> A) {
+    const int64_t K = D + H, n = B * K;
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t b = e / K, k = e % K;
+#pragma unroll
+        for (int p = 0; p < 2; ++p)
+            A.p[p][e] = k < D ? X.p[p][b * xw + (int64_t)t * D + k] : (hprev.p[p] ? hprev.p[p][b * H + (k - D)] : (T)0);
+    }
+}
+static __global__ void add_pair_kernel(CPair<T> a, CPair<T> b, int64_t n, Pair<T> c) {
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x)
+#pragma unroll
+        for (int p = 0; p < 2; ++p) c.p[p][e] = a.p[p][e] + b.p[p][e];
+}
+
 // out_p = (neg ? -in_p : in_p) + [p == 0] c   (public constants are added by party 0)
 static __global__ void affine_pair_kernel(CPair<T> in, int64_t n, T c, int neg, Pair<T> out) {
     for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x)
@@ -726,6 +771,25 @@ static psml_status forward(psml_model_s *m, const T *const X[2], const T *const 
     m->act[0].p[0] = (T *)X[0];
     m->act[0].p[1] = (T *)X[1];
     T *yo[2] = {out ? out[0] : m->yhat.p[0], out ? out[1] : m->yhat.p[1]};
+    if (m->d.kind == PSML_RNN) {
+        const int T = m->rnn_T;
+        const int64_t D = m->rnn_D, H = m->dims[1], K1 = m->rows[0], B = m->B;
+        for (int t = 1; t <= T; ++t) {
+            T_ *At[2] = {m->rnnA.p[0] + (t - 1) * B * K1, m->rnnA.p[1] + (t - 1) * B * K1};
+            const T_ *hp[2] = {t > 1 ? m->rnnH.p[0] + (t - 2) * B * H : nullptr, t > 1 ? m->rnnH.p[1] + (t - 2) * B * H : nullptr};
+            rnn_concat_kernel<<<ew_grid(B * K1), EW_THREADS, 0, s>>>(CPair<T_>{{X[0], X[1]}}, CPair<T_>{{hp[0], hp[1]}}, B, D,
+                                                                    H, (int64_t)m->dims[0], t - 1, Pair<T_>{{At[0], At[1]}});
+            PSML_LAUNCH_CHECK();
+            const T_ *Ac[2] = {At[0], At[1]};
+            PSML_TRY(mm(m, Ac, m->W[0].cp(), t, OP_FWD, 0, fw(m, 0), m->z[0].pp(), s));
+            T_ *ht[2] = {m->rnnH.p[0] + (t - 1) * B * H, m->rnnH.p[1] + (t - 1) * B * H};
+            T_ *dt[2] = {m->rnnD.p[0] + (t - 1) * B * H, m->rnnD.p[1] + (t - 1) * B * H};
+            PSML_TRY(relu(m, m->z[0].cp(), t, ht, dt, s));
+        }
+        const T_ *hT[2] = {m->rnnH.p[0] + (T - 1) * B * H, m->rnnH.p[1] + (T - 1) * B * H};
+        PSML_TRY(mm(m, hT, m->W[1].cp(), T + 1, OP_FWD, 0, fw(m, 1), m->z[1].pp(), s));
+        return eq9(m, m->z[1].cp(), T + 1, yo, Y, Y ? m->delta.pp() : nullptr, s);
+    }
     if (m->d.kind == PSML_SVM) {
         PSML_TRY(mm(m, m->act[0].cp(), m->W[0].cp(), 0, OP_FWD, 0, fw(m, 0), m->z[0].pp(), s));
         const int64_t n = m->B;
@@ -763,6 +827,34 @@ static psml_status backward(psml_model_s *m, cudaStream_t s) {
     T *g[2];
     if (m->d.kind == PSML_SVM)
         return mm(m, m->act[0].cp(), m->delta.cp(), 0, OP_GRADW, PSML_TRANS_A, 0, gradp(m, 0, g), s);
+    if (m->d.kind == PSML_RNN) {   // backpropagation through time (R25)
+        const int T = m->rnn_T;
+        const int64_t D = m->rnn_D, H = m->dims[1], K1 = m->rows[0], B = m->B;
+        const T_ *hT[2] = {m->rnnH.p[0] + (T - 1) * B * H, m->rnnH.p[1] + (T - 1) * B * H};
+        PSML_TRY(mm(m, hT, m->delta.cp(), T + 1, OP_GRADW, PSML_TRANS_A, 0, gradp(m, 1, g), s));
+        PSML_TRY(mm(m, m->delta.cp(), m->W[1].cp(), T + 1, OP_GRADIN, PSML_TRANS_B, fw(m, 1), m->tmp.pp(), s));
+        const T_ *dT[2] = {m->rnnD.p[0] + (T - 1) * B * H, m->rnnD.p[1] + (T - 1) * B * H};
+        PSML_TRY(had(m, m->tmp.cp(), dT, T, 1, m->delta.pp(), s));
+        T_ *g0[2];
+        gradp(m, 0, g0);
+        const T_ *Wh[2] = {m->W[0].p[0] + D * H, m->W[0].p[1] + D * H};   // W_h = rows D.. of W_1
+        for (int t = T; t >= 1; --t) {
+            const T_ *At[2] = {m->rnnA.p[0] + (t - 1) * B * K1, m->rnnA.p[1] + (t - 1) * B * K1};
+            PSML_TRY(mm(m, At, m->delta.cp(), t, OP_GRADW, PSML_TRANS_A, 0, t == T ? g0 : m->rnnG.pp(), s));
+            if (t < T) {   // gW_1 += A_t^T delta_t  (ring addition of untruncated shares)
+                add_pair_kernel<<<ew_grid(K1 * H), EW_THREADS, 0, s>>>(CPair<T_>{{g0[0], g0[1]}},
+                                                                      CPair<T_>{{m->rnnG.p[0], m->rnnG.p[1]}},
+                                                                      K1 * H, Pair<T_>{{g0[0], g0[1]}});
+                PSML_LAUNCH_CHECK();
+            }
+            if (t > 1) {
+                PSML_TRY(mm(m, m->delta.cp(), Wh, t, OP_GRADIN, PSML_TRANS_B, fw(m, 0), m->tmp.pp(), s));
+                const T_ *dp[2] = {m->rnnD.p[0] + (t - 2) * B * H, m->rnnD.p[1] + (t - 2) * B * H};
+                PSML_TRY(had(m, m->tmp.cp(), dp, t - 1, 1, m->delta.pp(), s));
+            }
+        }
+        return PSML_OK;
+    }
     if (m->d.kind == PSML_CNN) {
         // layer 2 (FC 64 -> 10)
         PSML_TRY(mm(m, m->act[2].cp(), m->delta.cp(), 2, OP_GRADW, PSML_TRANS_A, 0, gradp(m, 2, g), s));
@@ -798,7 +890,7 @@ static int item_index(const psml_model_s *m, int layer, int op, int slot) {
 }
 
 static bool fused_eligible(const psml_model_s *m) {
-    if (m->d.kind == PSML_CNN || m->d.kind == PSML_SVM || m->nl > UPD_MAX_LAYERS ||
+    if (m->d.kind == PSML_CNN || m->d.kind == PSML_SVM || m->d.kind == PSML_RNN || m->nl > UPD_MAX_LAYERS ||
         (int)m->ob.size() != (int)m->items[0].size())
         return false;
     for (int l = 0; l < m->nl; ++l)
@@ -1358,6 +1450,18 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
         m->cols = {desc->cnn_cout, desc->cnn_hidden, desc->cnn_classes};
         break;
     }
+    case PSML_RNN: {
+        const int64_t D = desc->dims[0], H = desc->dims[1], C = desc->dims[2];
+        if (D <= 0 || H <= 0 || C <= 0 || desc->rnn_steps <= 0 || desc->rnn_steps > 254)
+            return fail(PSML_ERR_SHAPE, "RNN: dims = {D, H, C} > 0 and 1 <= rnn_steps <= 254");
+        m->nl = 2;
+        m->rnn_T = desc->rnn_steps;
+        m->rnn_D = (int)D;
+        m->dims = {(int64_t)desc->rnn_steps * D, H, C};
+        m->rows = {D + H, H};
+        m->cols = {H, C};
+        break;
+    }
     default:
         return fail(PSML_ERR_INVALID, "unknown model kind");
     }
@@ -1396,6 +1500,13 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
     PSML_TRY(balloc(mp, m->yhat, B * m->dims[m->nl]));
     PSML_TRY(balloc(mp, m->delta, B * maxw));
     PSML_TRY(balloc(mp, m->tmp, B * std::max<int64_t>(maxw, 3)));   // SVM: margin, indicator, y (.) ind
+    if (m->d.kind == PSML_RNN) {
+        const int64_t T = m->rnn_T, H = m->dims[1];
+        PSML_TRY(balloc(mp, m->rnnA, T * B * m->rows[0]));
+        PSML_TRY(balloc(mp, m->rnnH, T * B * H));
+        PSML_TRY(balloc(mp, m->rnnD, T * B * H));
+        PSML_TRY(balloc(mp, m->rnnG, m->rows[0] * H));
+    }
     if (m->d.kind == PSML_CNN) {   // im2col column offsets (ch, ky, kx) -> ch*H*W + ky*W + kx
         const ConvGeom &g = m->g;
         std::vector<int32_t> off((size_t)g.C * g.k * g.k);
@@ -1927,7 +2038,8 @@ psml_status psml_party_forward_backward(psml_model m, int32_t party, psml_xport 
                                         uint32_t step_id, psml_stream stream) {
     if (!m || !x) return fail(PSML_ERR_INVALID, "null model or transport");
     if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
-    if (m->d.kind == PSML_SVM) return fail(PSML_ERR_UNSUPPORTED, "SVM: co-resident engine only");
+    if (m->d.kind == PSML_SVM || m->d.kind == PSML_RNN)
+        return fail(PSML_ERR_UNSUPPORTED, "SVM / RNN: co-resident engine only");
     PSML_TRY(check_ptrs({X_i, Y_i}));
     const int pool = (int)(step_id & 1);
     if (m->dealt_step[pool] != (int64_t)step_id || !m->dealt_full[pool])

@@ -18,7 +18,7 @@ STATUS = {0: "PSML_OK", 1: "PSML_ERR_INVALID", 2: "PSML_ERR_SHAPE", 3: "PSML_ERR
           4: "PSML_ERR_UNSUPPORTED", 5: "PSML_ERR_CUDA", 6: "PSML_ERR_NOMEM", 7: "PSML_ERR_STATE",
           8: "PSML_ERR_NCCL"}
 TRANS_A, TRANS_B, PAPER_FORM = 1, 2, 4
-LINREG, LOGREG, MLP, CNN, SVM = 0, 1, 2, 3, 4
+LINREG, LOGREG, MLP, CNN, SVM, RNN = 0, 1, 2, 3, 4, 5
 
 vp, i32, i64, u32, u64 = (ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64, ctypes.c_uint32,
                           ctypes.c_uint64)
@@ -44,7 +44,8 @@ class ModelDesc(ctypes.Structure):
                 ("lr_shift", i32), ("master_frac_bits", i32), ("dealer_seed", u64),
                 ("pair_id", u32), ("cnn_c", i32), ("cnn_h", i32), ("cnn_w", i32), ("cnn_k", i32),
                 ("cnn_cout", i32), ("cnn_hidden", i32), ("cnn_classes", i32),
-                ("fwd_frac_bits", i32 * 8), ("compare", i32), ("weight_decay_shift", i32)]
+                ("fwd_frac_bits", i32 * 8), ("compare", i32), ("weight_decay_shift", i32),
+                ("rnn_steps", i32)]
 
 
 # psml_exchange_fn (include/psml.h): (user, n, send[], recv[], bytes[], stream) -> 0 on success
@@ -514,11 +515,11 @@ class Model:
 
     def __init__(self, ctx, kind, dims=None, batch=128, lr_shift=14, master_frac_bits=27,
                  dealer_seed=0x50534D4C + 2, pair_id=0, cnn=(3, 32, 32, 5, 16, 64, 10),
-                 fwd_frac_bits=None, compare=0, weight_decay_shift=0):
+                 fwd_frac_bits=None, compare=0, weight_decay_shift=0, rnn_steps=0):
         d = ModelDesc()
         d.kind = kind
         dims = list(dims or ([784, 1] if kind in (LINREG, LOGREG, SVM) else [784, 128, 128, 10]))
-        d.n_layers = 3 if kind == CNN else len(dims) - 1
+        d.n_layers = 3 if kind == CNN else (2 if kind == RNN else len(dims) - 1)
         for i, v in enumerate(dims[:8]):
             d.dims[i] = v
         d.batch, d.lr_shift, d.master_frac_bits = batch, lr_shift, master_frac_bits
@@ -528,6 +529,7 @@ class Model:
             d.fwd_frac_bits[i] = v
         d.compare = compare                           # 0 A2B chain (R9), 1 FSS comparison (R22)
         d.weight_decay_shift = weight_decay_shift     # SVM weight decay (R24)
+        d.rnn_steps = rnn_steps                       # RNN sequence length (R25)
         self.ctx, self.desc, self.kind = ctx, d, kind
         h = vp()
         _call("psml_model_create", ctx.handle, ctypes.byref(d), ctypes.byref(h))

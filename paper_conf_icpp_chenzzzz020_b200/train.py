@@ -23,7 +23,9 @@ SHARE_SEED = DATA_SEED + 1
 DEALER_SEED = DATA_SEED + 2
 OP_SHARE = 7
 INIT_STEP = 0xFFFFFFFF
-KINDS = {"linreg": psml.LINREG, "logreg": psml.LOGREG, "mlp": psml.MLP, "cnn": psml.CNN, "svm": psml.SVM}
+KINDS = {"linreg": psml.LINREG, "logreg": psml.LOGREG, "mlp": psml.MLP, "cnn": psml.CNN, "svm": psml.SVM,
+         "rnn": psml.RNN}
+RNN_SHAPE = dict(dims=[32, 64, 10], rnn_steps=16)   # D, H, C and T (R25; synth.RNN_*)
 WD_SHIFT = {"svm": 16}   # weight decay lambda.eta = 2^-16 (R24)
 # forward-weight fractional bits per layer (R21); None = frac_bits for every layer
 FWD_BITS = {"cnn": [16, 20, 20]}
@@ -45,7 +47,9 @@ class SecureTrainer:
         self.master_ring = psml.Ring(64, master_frac_bits)
         self.pair_id = pair_id
         self.batch = batch
-        self.model = psml.Model(self.ctx, KINDS[task], dims=dims, batch=batch, lr_shift=lr_shift,
+        rnn = RNN_SHAPE if task == "rnn" else {}
+        self.model = psml.Model(self.ctx, KINDS[task], dims=dims or rnn.get("dims"), batch=batch, lr_shift=lr_shift,
+                                rnn_steps=rnn.get("rnn_steps", 0),
                                 master_frac_bits=master_frac_bits, dealer_seed=DEALER_SEED,
                                 pair_id=pair_id, fwd_frac_bits=FWD_BITS.get(task),
                                 compare={"a2b": 0, "fss": 1}[compare], weight_decay_shift=WD_SHIFT.get(task, 0))
@@ -54,6 +58,14 @@ class SecureTrainer:
             Wm = psml.share(self.ring, SHARE_SEED, call_id(0, INIT_STEP, layer, OP_SHARE, 2), w)
             self.model.set_master(layer, Wm)
         self.out_dim = self.model.layer_shape(self.model.n_layers - 1)[1]
+
+    def d_in(self):
+        """Features per input row: CNN 3x32x32, RNN T x D, else the first layer's fan-in."""
+        if self.task == "cnn":
+            return 3 * 32 * 32
+        if self.task == "rnn":
+            return RNN_SHAPE["rnn_steps"] * RNN_SHAPE["dims"][0]
+        return self.model.layer_shape(0)[0]
 
     # --- client side -----------------------------------------------------------------------
     def _client_share(self, X, Y, step, outX=None, outY=None):
@@ -84,7 +96,7 @@ class SecureTrainer:
         """Capture deal + online step (+ update) into CUDA graph(s) on a side stream; the batch is
         shared into fixed buffers before each replay (graph_step).  pipelined: the dealer of the
         next step runs concurrently with the online phase of this one (double-buffered pools)."""
-        d_in = self.model.layer_shape(0)[0] if self.task != "cnn" else 3 * 32 * 32
+        d_in = self.d_in()
         self.Xbuf = psml.empty_pair((self.batch, d_in), 64)
         self.Ybuf = psml.empty_pair((self.batch, self.out_dim), 64)
         for t in self.Xbuf + self.Ybuf:
@@ -210,7 +222,7 @@ class PartyTrainer(SecureTrainer):
     def capture_party(self, pipelined=True):
         """Capture this party's whole step (dealer [pipelined], online phase with its exchanges,
         gradient all-reduce, update) into CUDA graph(s) reading fixed share buffers."""
-        d_in = self.model.layer_shape(0)[0] if self.task != "cnn" else 3 * 32 * 32
+        d_in = self.d_in()
         self.Xi = torch.zeros((self.batch, d_in), dtype=torch.uint64, device="cuda")
         self.Yi = torch.zeros((self.batch, self.out_dim), dtype=torch.uint64, device="cuda")
         self.gstream = torch.cuda.Stream()

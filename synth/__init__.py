@@ -29,8 +29,12 @@ BLOCK = 128
 MNIST_FEATURES = 784
 CIFAR_SHAPE = (3, 32, 32)
 CIFAR_FEATURES = 3 * 32 * 32
+# SYNTHETIC sequences for the RNN ("RNN does not apply to images, so we only use our
+# generated dataset, SYNTHETIC"): T steps of D dense 8-bit features; R25.
+RNN_T, RNN_D, RNN_H, RNN_C = 16, 32, 64, 10
+SEQ_FEATURES = RNN_T * RNN_D
 
-_KIND = {"mnist": 1, "cifar": 2}
+_KIND = {"mnist": 1, "cifar": 2, "seq": 3}
 
 
 def _block_pixels(kind, b, seed):
@@ -40,13 +44,14 @@ def _block_pixels(kind, b, seed):
         keep = rng.random((BLOCK, MNIST_FEATURES)) < 0.19
         k = np.minimum(np.floor(x * 255.0), 254.0).astype(np.uint8) + 1   # 1..255
         return np.where(keep, k, 0).astype(np.uint8)
-    return np.minimum(np.floor(rng.random((BLOCK, CIFAR_FEATURES)) * 256.0), 255.0).astype(np.uint8)
+    width = CIFAR_FEATURES if kind == "cifar" else SEQ_FEATURES
+    return np.minimum(np.floor(rng.random((BLOCK, width)) * 256.0), 255.0).astype(np.uint8)
 
 
 def pixels(kind, start, count, seed=DATA_SEED):
     """8-bit pixels of rows [start, start+count) of the synthetic dataset `kind`."""
     if count <= 0:
-        width = MNIST_FEATURES if kind == "mnist" else CIFAR_FEATURES
+        width = {"mnist": MNIST_FEATURES, "cifar": CIFAR_FEATURES, "seq": SEQ_FEATURES}[kind]
         return np.zeros((0, width), dtype=np.uint8)
     b0, b1 = start // BLOCK, (start + count - 1) // BLOCK
     blocks = np.concatenate([_block_pixels(kind, b, seed) for b in range(b0, b1 + 1)], axis=0)
@@ -87,6 +92,12 @@ def cnn_teacher(seed=TEACHER_SEED, cout=16, k=5, hidden=64, classes=10):
             rng.normal(0.0, 1.0, size=(hidden, classes)) / np.sqrt(hidden)]
 
 
+def rnn_teacher(seed=TEACHER_SEED):
+    rng = np.random.default_rng([seed, 5])
+    return [rng.normal(0.0, 1.0, size=(RNN_D + RNN_H, RNN_H)) / np.sqrt(RNN_D + RNN_H),
+            rng.normal(0.0, 1.0, size=(RNN_H, RNN_C)) / np.sqrt(RNN_H)]
+
+
 def _patches(X, k=5):
     """(B, 3072) -> (B*28*28, 75) patch matrix for the teacher conv (label generation only)."""
     B = X.shape[0]
@@ -121,11 +132,17 @@ def labels(task, X):
         Wc, W1, W2 = cnn_teacher()
         h = relu(_patches(X) @ Wc).reshape(X.shape[0], -1)
         return _one_hot(relu(h @ W1) @ W2)
+    if task == "rnn":
+        W1, Wo = rnn_teacher()
+        h = np.zeros((X.shape[0], RNN_H))
+        for t in range(RNN_T):
+            h = relu(np.concatenate([X[:, t * RNN_D:(t + 1) * RNN_D], h], axis=1) @ W1)
+        return _one_hot(h @ Wo)
     raise ValueError(task)
 
 
-TASK_DATA = {"linreg": "mnist", "logreg": "mnist", "svm": "mnist", "mlp": "mnist", "cnn": "cifar"}
-TASK_ROWS = {"mnist": 60000, "cifar": 50000}
+TASK_DATA = {"linreg": "mnist", "logreg": "mnist", "svm": "mnist", "mlp": "mnist", "cnn": "cifar", "rnn": "seq"}
+TASK_ROWS = {"mnist": 60000, "cifar": 50000, "seq": 60000}
 
 
 def batch(task, step, batch_size=BLOCK, pair=0, n_pairs=1, seed=DATA_SEED):
@@ -145,7 +162,7 @@ def batch_u8(task, step, batch_size=BLOCK, pair=0, n_pairs=1, seed=DATA_SEED):
     start = ((step * n_pairs + pair) * batch_size) % (TASK_ROWS[kind] - batch_size + 1)
     q = pixels(kind, start, batch_size, seed)
     Y = labels(task, q.astype(np.float64) / 255.0)
-    if task in ("mlp", "cnn"):
+    if task in ("mlp", "cnn", "rnn"):
         return q, np.argmax(Y, axis=1).astype(np.uint8)
     return q, Y
 
@@ -160,6 +177,8 @@ def init_weights(task, dims=None, seed=INIT_SEED):
         shapes = list(zip(dims[:-1], dims[1:]))
     elif task == "cnn":
         shapes = [(75, 16), (12544, 64), (64, 10)]
+    elif task == "rnn":
+        shapes = [(RNN_D + RNN_H, RNN_H), (RNN_H, RNN_C)]
     else:
         raise ValueError(task)
     rng = np.random.default_rng([seed, 7])

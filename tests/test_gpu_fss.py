@@ -85,7 +85,7 @@ def _compare_shares(tr, om):
         assert np.array_equal(to_np(g1).reshape(om.Wm[layer][1].shape), om.Wm[layer][1]), layer
 
 
-@pytest.mark.parametrize("task,steps", [("logreg", 2), ("svm", 2), ("mlp", 2)])
+@pytest.mark.parametrize("task,steps", [("logreg", 2), ("svm", 2), ("mlp", 2), ("rnn", 1)])
 def test_training_with_fss_comparison_bitexact(P, task, steps):
     """Every ReLU / Eq. 9 of the step through the one-round FSS comparison: eager steps and
     CUDA-graph replays (dealer inside the graph) bit-exact vs the oracle's protocol."""

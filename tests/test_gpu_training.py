@@ -30,7 +30,7 @@ def _compare_shares(tr, om):
         assert np.array_equal(to_np(g1).reshape(om.Wm[layer][1].shape), om.Wm[layer][1]), layer
 
 
-@pytest.mark.parametrize("task,steps", [("linreg", 3), ("logreg", 3), ("svm", 3), ("mlp", 3), ("cnn", 1)])
+@pytest.mark.parametrize("task,steps", [("linreg", 3), ("logreg", 3), ("svm", 3), ("mlp", 3), ("rnn", 2), ("cnn", 1)])
 def test_training_bitexact_vs_oracle(T, task, steps):
     Wi = synth.init_weights(task)
     tr = T.SecureTrainer(task, Wi, backend=1)
@@ -45,7 +45,7 @@ def test_training_bitexact_vs_oracle(T, task, steps):
     tr.close()
 
 
-@pytest.mark.parametrize("task", ["mlp", "logreg", "svm"])
+@pytest.mark.parametrize("task", ["mlp", "logreg", "svm", "rnn"])
 def test_inference_bitexact_vs_oracle(T, task):
     Wi = synth.init_weights(task)
     tr = T.SecureTrainer(task, Wi, backend=1)
@@ -60,7 +60,7 @@ def test_inference_bitexact_vs_oracle(T, task):
     tr.close()
 
 
-@pytest.mark.parametrize("task,tol_log2", [("linreg", -12), ("logreg", -12), ("svm", -12), ("mlp", -12)])
+@pytest.mark.parametrize("task,tol_log2", [("linreg", -12), ("logreg", -12), ("svm", -12), ("mlp", -12), ("rnn", -12)])
 def test_one_epoch_within_2pow_minus12_of_fp64(T, task, tol_log2):
     """BASELINE north_star: decoded weights within 2^-12 of plaintext fp64 after one epoch
     (60000 MNIST-shaped rows, batch 128, 468 steps, R13-R15)."""

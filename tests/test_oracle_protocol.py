@@ -328,3 +328,34 @@ def test_comparison_lt0_edges(orc, compare):
     t0 = orc.prg(64, 21, orc.tag("tt"), 0, t.size)
     got = P.comparison_lt0((t0, t - t0), 0, 9, 0, compare)
     assert np.array_equal(got[0] + got[1], (t.view(np.int64) < 0).astype(np.uint64))
+
+
+def test_rnn_training_tracks_fp64_and_inference():
+    """Elman RNN with BPTT (R25) on SYNTHETIC sequences: decoded master weights after 6
+    steps vs the fp64 BPTT of oracle/plain.py, zero comparison mismatches / truncation failures,
+    and the secure forward vs the plaintext forward."""
+    task = "rnn"
+    Wi = synth.init_weights(task)
+    m, pm = P.Model(task, Wi), plain.PlainModel(task, Wi)
+    P.diag_reset(True)
+    try:
+        for s in range(6):
+            X, Y = synth.batch(task, s)
+            P.train_step(m, X, Y, s)
+            pm.step(X, Y)
+        d = dict(P.DIAG)
+    finally:
+        P.diag_reset(False)
+    assert d["msb_fail"] == 0 and d["trunc_fail"] == 0, d
+    err = max(np.abs(a - b).max() for a, b in zip(m.decoded_master(), pm.W))
+    assert err < 2.0 ** -15, np.log2(err)
+    from oracle import core
+    X, Y = synth.batch(task, 40)
+    Xs, _ = P.share_batch(X, Y, 40)
+    got = core.decode(core.reconstruct(*P.infer(m, Xs, step=900)))
+    Xq = plain.q(X, P.F)
+    W1, Wo = pm.W
+    h = np.zeros((X.shape[0], 64))
+    for t in range(16):
+        h = np.maximum(np.concatenate([Xq[:, 32 * t:32 * (t + 1)], h], axis=1) @ W1, 0.0)
+    assert np.abs(got - plain.eq9(h @ Wo)).max() < 2.0 ** -8
