@@ -441,6 +441,20 @@ psml_status psml_dp_destroy(psml_dp dp);
 psml_status psml_dp_size(psml_dp dp, int32_t *size);
 psml_status psml_dp_allreduce(psml_dp dp, void *buf, int64_t n, int32_t l, psml_stream stream);
 
+/* Per-party context (one ctx per party per GPU per process).  The context carries
+ * this party, its pair transport (psml_xport_*_create, caller-owned, must outlive the ctx) and
+ * its data-parallel communicator (nullable).  psml_secure_matmul_party is the collective
+ * one-party Beaver product: both parties call it with identical shapes and flags in the same
+ * order; it masks E_i = op(A)_i - U_i, F_i = op(B)_i - V_i (Eq. 4), exchanges them through the
+ * pair transport (Eq. 5), and computes C_i = i.E.F + E.V_i + U_i.F + Z_i (Eq. 8 shape) with
+ * SecureML truncation by trunc_bits -- bit-identical to psml_secure_matmul's party-i share.
+ * All pointers are this party's device buffers; flags: PSML_TRANS_A / PSML_TRANS_B. */
+psml_status psml_ctx_create_party(psml_ring ring, int32_t gemm_backend, int32_t party, psml_xport pair, psml_dp dp,
+                                  psml_ctx *out);
+psml_status psml_secure_matmul_party(psml_ctx ctx, const void *A_i, const void *B_i, const void *U_i, const void *V_i,
+                                     const void *Z_i, int64_t M, int64_t K, int64_t N, int32_t flags,
+                                     int32_t trunc_bits, void *C_i, psml_stream stream);
+
 /* Party `party`'s half of one training step (LINREG / LOGREG / MLP / CNN): X_i: batch x d_0
  * (CNN: batch x C*H*W), Y_i: batch x d_L, this party's shares (device).  The model's dealer
  * pool must hold the step's material (psml_model_deal; in this simulation each party's process

@@ -202,11 +202,61 @@ psml_status psml_ctx_create(psml_ring ring, int32_t gemm_backend, psml_ctx *out)
     return PSML_OK;
 }
 
+psml_status Ctx::ensure_msg(size_t bytes) {
+    if (bytes <= msg_bytes) return PSML_OK;
+    if (msg) {
+        PSML_CUDA_TRY(cudaDeviceSynchronize());
+        PSML_CUDA_TRY(cudaFree(msg));
+        msg = nullptr;
+        msg_bytes = 0;
+    }
+    if (cudaMalloc(&msg, bytes) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(PSML_ERR_NOMEM, "message buffer allocation failed");
+    }
+    msg_bytes = bytes;
+    return PSML_OK;
+}
+
+psml_status psml_ctx_create_party(psml_ring ring, int32_t gemm_backend, int32_t party, psml_xport pair, psml_dp dp,
+                                  psml_ctx *out) {
+    if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
+    if (!pair) return fail(PSML_ERR_INVALID, "a per-party context needs its pair transport");
+    PSML_TRY(psml_ctx_create(ring, gemm_backend, out));
+    Ctx *c = reinterpret_cast<Ctx *>(*out);
+    c->party = party;
+    c->xport = pair;
+    c->dp = dp;
+    return PSML_OK;
+}
+
+psml_status psml_secure_matmul_party(psml_ctx ctx, const void *A_i, const void *B_i, const void *U_i, const void *V_i,
+                                     const void *Z_i, int64_t M, int64_t K, int64_t N, int32_t flags,
+                                     int32_t trunc_bits, void *C_i, psml_stream stream) {
+    if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
+    Ctx *c = reinterpret_cast<Ctx *>(ctx);
+    if (c->party < 0 || !c->xport) return fail(PSML_ERR_STATE, "not a per-party context (psml_ctx_create_party)");
+    if (M <= 0 || K <= 0 || N <= 0) return fail(PSML_ERR_SHAPE, "M, K, N must be positive");
+    const size_t w = c->ring.l / 8;
+    PSML_TRY(c->ensure_msg(w * 2 * (size_t)(M * K + K * N) + 512));
+    uint8_t *b = (uint8_t *)c->msg;
+    void *Es = b, *Fs = b + w * M * K;
+    void *Er = b + w * (M * K + K * N), *Fr = b + w * (2 * M * K + K * N);
+    // round 1 (Eq. 4), the exchange of E_i and F_i (Eq. 5) through the pair transport, round 2
+    PSML_TRY(psml_beaver_mask(ctx, c->party, A_i, B_i, U_i, V_i, M, K, N, flags, Es, Fs, stream));
+    const void *snd[2] = {Es, Fs};
+    void *rcv[2] = {Er, Fr};
+    const int64_t bytes[2] = {(int64_t)w * M * K, (int64_t)w * K * N};
+    PSML_TRY(psml_xport_exchange(c->xport, 2, snd, rcv, bytes, stream));
+    return psml_beaver_open_matmul(ctx, c->party, Es, Er, Fs, Fr, U_i, V_i, Z_i, M, K, N, trunc_bits, C_i, stream);
+}
+
 psml_status psml_ctx_destroy(psml_ctx ctx) {
     if (!ctx) return PSML_OK;
     Ctx *c = reinterpret_cast<Ctx *>(ctx);
+    if (c->ws || c->msg) cudaDeviceSynchronize();
+    if (c->msg) cudaFree(c->msg);
     if (c->ws) {
-        cudaDeviceSynchronize();
         cudaFree(c->ws);
     }
     delete c;
@@ -415,6 +465,37 @@ psml_status psml_msb_dealer(psml_ring ring, uint64_t seed, uint64_t call_id, int
 // ------------------------------------------------------------------------------------------------
 // server side
 // ------------------------------------------------------------------------------------------------
+// Config 1 (one linear-regression minibatch, A M x K . B K x 1) in ONE launch: a warp per output
+// row, both parties.  Each warp re-derives the opened F = (B_0 - V_0) + (B_1 - V_1) of its K
+// columns (K words, L2-resident) and the opened row E_m = (A_0 - U_0) + (A_1 - U_1) (Eqs. 4-5),
+// then C_p[m] = p E_m.F + E_m.V_p + U_p[m].F + Z_p[m] (BJ form, the Eq. 8 K-concatenation), and
+// the SecureML truncation -- the mask, open and GEMV rounds of the co-resident pair fused.
+template <typename T>
+__global__ void __launch_bounds__(256) beaver_gemv_kernel(CPair<T> A, CPair<T> B, CPair<T> U, CPair<T> V, CPair<T> Z,
+                                                          int64_t M, int64_t K, int trunc, Pair<T> C) {
+    const int lane = threadIdx.x & 31;
+    const int64_t row = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (row >= M) return;
+    T acc0 = 0, acc1 = 0;
+    const T *a0 = A.p[0] + row * K, *a1 = A.p[1] + row * K, *u0 = U.p[0] + row * K, *u1 = U.p[1] + row * K;
+    for (int64_t k = lane; k < K; k += 32) {
+        const T f = (B.p[0][k] - V.p[0][k]) + (B.p[1][k] - V.p[1][k]);
+        const T uu0 = __ldcs(u0 + k), uu1 = __ldcs(u1 + k);
+        const T e = (__ldcs(a0 + k) - uu0) + (__ldcs(a1 + k) - uu1);
+        acc0 += e * V.p[0][k] + uu0 * f;
+        acc1 += e * f + e * V.p[1][k] + uu1 * f;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        acc0 += __shfl_xor_sync(0xffffffffu, acc0, o);
+        acc1 += __shfl_xor_sync(0xffffffffu, acc1, o);
+    }
+    if (lane == 0) {
+        C.p[0][row] = trunc_share<T>(acc0 + Z.p[0][row], 0, trunc);
+        C.p[1][row] = trunc_share<T>(acc1 + Z.p[1][row], 1, trunc);
+    }
+}
+
 template <typename T>
 static psml_status secure_matmul_t(Ctx *c, const void *const A[2], const void *const B[2], const void *const U[2],
                                    const void *const V[2], const void *const Z[2], int64_t M, int64_t K, int64_t N,
@@ -427,6 +508,14 @@ static psml_status secure_matmul_t(Ctx *c, const void *const A[2], const void *c
     if (!tr && !(flags & PSML_PAPER_FORM) && c->use_tc(M, 2 * K, N)) {
         psml_status st = tc_beaver_matmul<T>(c, a, b, u, v, z, M, K, N, flags, trunc, cc, s);
         if (st != PSML_ERR_UNSUPPORTED) return st;
+    }
+    if (!tr && flags == 0 && N == 1 && K <= 65536) {   // config 1: one fused launch
+        ProfScope prof(PROF_GEMM, s, (double)M * 2 * K * 2);
+        beaver_gemv_kernel<T><<<(unsigned)((M * 32 + 255) / 256), 256, 0, s>>>(
+            CPair<T>{{a[0], a[1]}}, CPair<T>{{b[0], b[1]}}, CPair<T>{{u[0], u[1]}}, CPair<T>{{v[0], v[1]}},
+            CPair<T>{{z[0], z[1]}}, M, K, trunc, Pair<T>{{cc[0], cc[1]}});
+        PSML_LAUNCH_CHECK();
+        return PSML_OK;
     }
     const int64_t words = beaver_ws_words<T>(M, K, N);
     PSML_TRY(c->ensure_ws(sizeof(T) * words));

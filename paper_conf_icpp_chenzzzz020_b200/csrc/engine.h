@@ -19,6 +19,13 @@ struct Ctx {
     void *ws = nullptr;
     size_t ws_bytes = 0;
     psml_status ensure_ws(size_t bytes);
+    // per-party context (psml_ctx_create_party): this party, its pair transport, its DP group
+    int party = -1;                 // -1: co-resident pair engine
+    psml_xport xport = nullptr;
+    psml_dp dp = nullptr;
+    void *msg = nullptr;            // the party's send / receive message buffers
+    size_t msg_bytes = 0;
+    psml_status ensure_msg(size_t bytes);
     // tcgen05 limb GEMM pays once a party's product has >= 2^25 ring MACs (measured on B200:
     // 128x1568x128 is 2x faster on CUDA cores, 12544x256x64 1.5x and 1024^3 10x faster on tcgen05;
     // tools/mm_prof.py).

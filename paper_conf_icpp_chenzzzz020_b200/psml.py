@@ -117,6 +117,8 @@ _SIGS = {
     "psml_dp_size": (i32, [vp, vp]),
     "psml_dp_allreduce": (i32, [vp, vp, i64, i32, vp]),
     "psml_party_train_step": (i32, [vp, i32, vp, vp, vp, vp, u32, vp]),
+    "psml_ctx_create_party": (i32, [Ring, i32, i32, vp, vp, vp]),
+    "psml_secure_matmul_party": (i32, [vp, vp, vp, vp, vp, vp, i64, i64, i64, i32, i32, vp, vp]),
     "psml_fss_material_words": (i64, [Ring, i64]),
     "psml_fss_dealer": (i32, [Ring, u64, u64, i64, P2, vp]),
     "psml_secure_drelu_fss": (i32, [vp, P2, i64, P2, P2, vp, vp]),
@@ -245,11 +247,18 @@ def device_info():
 class Ctx:
     """psml_ctx: one per GPU and host thread.  backend: 0 auto, 1 CUDA-core, 2 tcgen05."""
 
-    def __init__(self, l=64, frac_bits=13, backend=0):
+    def __init__(self, l=64, frac_bits=13, backend=0, party=None, xport=None, dp=None):
+        """party/xport/dp: a per-party context (psml_ctx_create_party) for psml_secure_matmul_party."""
         self.ring = Ring(l, frac_bits)
         self.l = l
+        self.party = party
+        self._keep = (xport, dp)   # the transport / communicator must outlive the context
         h = vp()
-        _call("psml_ctx_create", self.ring, backend, ctypes.byref(h))
+        if party is None:
+            _call("psml_ctx_create", self.ring, backend, ctypes.byref(h))
+        else:
+            _call("psml_ctx_create_party", self.ring, backend, party, xport.handle, dp.handle if dp else None,
+                  ctypes.byref(h))
         self.handle = h
 
     def close(self):
@@ -372,6 +381,14 @@ def secure_matmul(ctx, A, B, U, V, Z, M, K, N, flags=0, trunc=0, out=None, trace
           M, K, N, flags, trunc, _pair(C), ctypes.byref(tr) if tr is not None else None,
           _stream(stream))
     return (C, tr_t) if trace else C
+
+
+def secure_matmul_party(ctx, A_i, B_i, U_i, V_i, Z_i, M, K, N, flags=0, trunc=0, out=None, stream=None):
+    """Collective one-party Beaver product through the ctx's pair transport (per-party ctx)."""
+    C = out if out is not None else torch.empty((M, N), dtype=dtype_of(ctx.l), device="cuda")
+    _call("psml_secure_matmul_party", ctx.handle, _ptr(A_i), _ptr(B_i), _ptr(U_i), _ptr(V_i), _ptr(Z_i), M, K, N,
+          flags, trunc, _ptr(C), _stream(stream))
+    return C
 
 
 def beaver_mask(ctx, party, A_i, B_i, U_i, V_i, M, K, N, flags=0, stream=None):

@@ -155,6 +155,26 @@ def test_secure_matmul_bitexact(P, orc, ctx, shape, flags):
         assert np.array_equal(to_np(T[k]), tr[k]), k
 
 
+@pytest.mark.parametrize("shape", [(128, 784, 1), (784, 128, 1), (1, 16, 1), (3, 5, 1), (300, 2049, 1)])
+@pytest.mark.parametrize("trunc", [0, 13])
+def test_secure_matmul_gemv_single_launch(P, orc, ctx, shape, trunc):
+    """Config 1 (N = 1, untraced): the mask, open and GEMV rounds fused into one launch
+    (beaver_gemv_kernel) -- bit-exact vs the oracle."""
+    l = ctx.l
+    M, K, N = shape
+    a = _rand(orc, l, M * K, 30 + M).reshape(M, K)
+    b = _rand(orc, l, K * N, 40 + K).reshape(K, N)
+    A, B = orc.share(a, SEED + 1, 3, l), orc.share(b, SEED + 1, 4, l)
+    trip = orc.triplet_gen(SEED + 2, 5, M, K, N, l)
+    W0, W1 = orc.beaver_matmul(A, B, trip, trunc=trunc, l=l)
+    td = [to_dev(t, l) for t in trip]
+    n0 = P.kernel_launch_count()
+    C = P.secure_matmul(ctx, pair_dev(A, l), pair_dev(B, l), td[0:2], td[2:4], td[4:6], M, K, N, trunc=trunc)
+    torch.cuda.synchronize()
+    assert P.kernel_launch_count() - n0 == 1
+    assert np.array_equal(to_np(C[0]), W0) and np.array_equal(to_np(C[1]), W1)
+
+
 @pytest.mark.parametrize("shape", [(4, 4, 4), (33, 70, 19), (128, 784, 128)])
 def test_secure_matmul_paper_form(P, orc, ctx, shape):
     l = ctx.l

@@ -55,6 +55,43 @@ def _party(rank, port, l, outdir):
     dist.destroy_process_group()
 
 
+def _party_ctx(rank, port, l, outdir):
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    from paper_conf_icpp_chenzzzz020_b200 import psml
+    from paper_conf_icpp_chenzzzz020_b200.parallel import make_transport
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=2)
+    torch.cuda.set_device(0)
+    dt = np.uint64 if l == 64 else np.uint32
+    dev = lambda x: torch.from_numpy(np.ascontiguousarray(x.astype(dt))).cuda()  # noqa: E731
+    xp = make_transport(rank, 1 - rank, kind="peer", capacity_bytes=4 << 20)
+    for ci, ((M, K, N), flags, backend) in enumerate(CASES):
+        A, B, trip = _inputs(l, M, K, N, flags)
+        ctx = psml.Ctx(l=l, backend=backend, party=rank, xport=xp)
+        C = psml.secure_matmul_party(ctx, dev(A[rank]), dev(B[rank]), dev(trip[rank]), dev(trip[2 + rank]),
+                                     dev(trip[4 + rank]), M, K, N, flags=flags, trunc=13)
+        np.save(os.path.join(outdir, f"c{ci}_{rank}.npy"), C.cpu().numpy().astype(np.uint64))
+        ctx.close()
+    xp.close()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("l", [64, 32])
+def test_per_party_ctx_secure_matmul(tmp_path, l):
+    """psml_ctx_create_party + psml_secure_matmul_party (SURVEY §8(b) one-party collective call):
+    the exchange goes through the library's peer-memory transport; bit-exact vs the oracle."""
+    from oracle import core as orc
+    mp.spawn(_party_ctx, args=(_free_port(), l, str(tmp_path)), nprocs=2, join=True)
+    for ci, ((M, K, N), flags, _) in enumerate(CASES):
+        A, B, trip = _inputs(l, M, K, N, flags)
+        opA = [np.ascontiguousarray(t.T) if flags & 1 else t for t in A]
+        opB = [np.ascontiguousarray(t.T) if flags & 2 else t for t in B]
+        W = orc.beaver_matmul(opA, opB, trip, trunc=13, l=l)
+        for p in range(2):
+            assert np.array_equal(np.load(tmp_path / f"c{ci}_{p}.npy"), W[p]), (ci, p)
+
+
 @pytest.mark.parametrize("l", [64, 32])
 def test_split_deployment_matches_oracle(tmp_path, l):
     from oracle import core as orc
