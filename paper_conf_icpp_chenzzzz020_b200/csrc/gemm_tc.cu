@@ -605,8 +605,7 @@ static psml_status launch_gemm(TcParams<typename Cfg<l>::T> P, int64_t Mp, int64
     int kbs = (nkb + splits - 1) / splits;
     splits = (nkb + kbs - 1) / kbs;
     P.kb_per_split = kbs;
-    static const int dbg = getenv("PSML_TC_DEBUG") ? atoi(getenv("PSML_TC_DEBUG")) : 0;
-    P.debug = dbg;
+    P.debug = 0;
     const int final_mode = P.mode;
     if (splits > 1) {
         if (!partial || partial_words < P.M * P.N * P.nparty)

@@ -520,14 +520,9 @@ psml_status tc_seg_group(const SegArgs<uint64_t> *jobs, int njobs, cudaStream_t 
 #ifdef TCSEG_TIMING
     if (const char *e = getenv("PSML_TCSEG_MMAS")) g.debug_mmas = atoi(e);
 #endif
-    // K split: double ks while the grid stays within sm_count / fill CTAs (PSML_TCSEG_FILL,
-    // default 2: half the SMs, the rest stays with the dealer branch) and each split keeps >= 2
-    // K blocks
-    static int fill = -1;
-    if (fill < 0) {
-        const char *e = getenv("PSML_TCSEG_FILL");
-        fill = e ? std::max(1, atoi(e)) : 2;
-    }
+    // K split: double ks while the grid stays within half the SMs (the rest stays with the
+    // dealer branch) and each split keeps >= 2 K blocks
+    const int fill = 2;
     int ks = 1;
     while (ks < max_ks && tiles * ks * 2 * fill <= 2 * sm_count && nkb_max >= ks * 2) ks *= 2;
     g.ks = ks;

@@ -428,13 +428,11 @@ static psml_status deal_item(psml_model_s *m, DealItem &it, uint32_t step, cudaS
 // Work lists of the fused dealer for items[pool] (step field of the call ids filled in on device).
 static psml_status build_plan(psml_model_s *m, int pool, bool infer_only) {
     DealPlan &P = m->plan[pool][infer_only ? 1 : 0];
-    {   // cluster split of the dealer's grouped Z = U V launch (PSML_DEAL_KS; default 4)
-        const char *e = getenv("PSML_DEAL_KS");
-        const int v = e ? atoi(e) : 4;
-        P.gemm_ks = (v == 1 || v == 2 || v == 4 || v == 8) ? v : 4;
-        const char *t = getenv("PSML_DEAL_TILE");   // 64: fewer, more ALU-efficient dealer CTAs
-        P.gemm_big = t && atoi(t) == 64;
-    }
+    // cluster split of the dealer's grouped Z = U V launch: 4 (measured vs 2 and 8: 919K vs
+    // 895K / 897K samples/s); 32 x 32 tiles (64 x 64 tiles measured 720K: their CTAs crowd out the
+    // online chain)
+    P.gemm_ks = 4;
+    P.gemm_big = false;
     const int gBM = P.gemm_big ? ClDealer::BM : ClDefault::BM, gBN = P.gemm_big ? ClDealer::BN : ClDefault::BN;
     const int gBK = P.gemm_big ? ClDealer::BK : ClDefault::BK;
     std::vector<PrgJob> pjm, pjr;   // matrix-triplet streams, then the rest
@@ -541,15 +539,9 @@ static psml_status deal_prg_launch(psml_model_s *m, const DealPlan &P, int j0, i
                                    cudaStream_t s, bool second = false) {
     if (j1 <= j0 || b1 <= b0) return PSML_OK;
     // a bounded grid (grid-stride): the PRG work runs beside the online phase instead of
-    // occupying every SM's register file ahead of it (PSML_DEAL_CTAS per SM; 0 = full grid;
-    // PSML_DEAL_CTAS2 for the second dealer branch)
-    static int per_sm1 = -1, per_sm2 = -1;
-    if (per_sm1 < 0) {
-        const char *e = getenv("PSML_DEAL_CTAS");
-        per_sm1 = e ? atoi(e) : 4;   // measured best of {1, 2, 4, full} (tools/gpu44.sh)
-        const char *e2 = getenv("PSML_DEAL_CTAS2");
-        per_sm2 = e2 ? atoi(e2) : std::min(per_sm1, 2);   // tools/gpu92.sh: 2 best of {2, 3, 4}
-    }
+    // occupying every SM's register file ahead of it
+    const int per_sm1 = 4;   // CTAs per SM, measured best of {1, 2, 4, full grid}
+    const int per_sm2 = 2;   // second branch: best of {2, 3, 4}
     // (the CNN's dealer is most of its step: both of its branches keep the full budget -- 56.3K vs
     // 54.7K samples/s with the MLP's split)
     const int per_sm = (second && m->d.kind != PSML_CNN) ? per_sm2 : per_sm1;
@@ -1533,11 +1525,9 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
         // work fills the SMs they leave idle (PSML_PRIO=0 disables)
         int lo = 0, hi = 0;
         PSML_CUDA_TRY(cudaDeviceGetStreamPriorityRange(&lo, &hi));
-        // PSML_DEAL_PRIO1: priority of the first dealer branch (matrix-triplet PRG + Z = U V, which
-        // the step's end waits for) as steps above the lowest; default the lowest
-        int p1 = lo;
-        if (const char *e = getenv("PSML_DEAL_PRIO1")) p1 = std::max(hi, lo - std::max(0, atoi(e)));
-        PSML_CUDA_TRY(cudaStreamCreateWithPriority(&m->side, cudaStreamNonBlocking, p1));
+        // both dealer branches at the lowest priority (raising the first one 1-3 steps measured
+        // 900K vs 914K samples/s)
+        PSML_CUDA_TRY(cudaStreamCreateWithPriority(&m->side, cudaStreamNonBlocking, lo));
         PSML_CUDA_TRY(cudaStreamCreateWithPriority(&m->side2, cudaStreamNonBlocking, lo));
         PSML_CUDA_TRY(cudaStreamCreateWithPriority(&m->hi, cudaStreamNonBlocking, hi));
         PSML_CUDA_TRY(cudaStreamCreateWithPriority(&m->gw, cudaStreamNonBlocking, hi));
@@ -1724,14 +1714,7 @@ static psml_status party_reduce_update(psml_model_s *m, int party, psml_dp dp, c
 // One captured step for online pool `pool`.  Non-pipelined: [dealer(pool)] -> online -> [update].
 // Pipelined: online(pool) -> [update] on `s`, concurrently dealer(1 - pool) for the NEXT step on the
 // side stream (fork/join inside the capture), reading the step word = step + 1.
-static bool use_prio() {
-    static int v = -1;
-    if (v < 0) {
-        const char *e = getenv("PSML_PRIO");
-        v = (e && e[0] == '0') ? 0 : 1;
-    }
-    return v == 1;
-}
+static bool use_prio() { return true; }   // stream priorities in the pipelined graph (865K -> 914K)
 
 static psml_status capture_one(psml_model_s *m, int pool, const T *const X[2], const T *const Y[2], int flags,
                                cudaStream_t s, cudaGraphExec_t *out, int64_t *kernels) {

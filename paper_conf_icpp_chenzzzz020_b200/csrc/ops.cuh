@@ -373,14 +373,7 @@ psml_status msb_chain(const T *const x[2], int64_t n, const T *const mat[2], int
     o.em.n = 0;
     if (em) o.em = *em;
     if (chain_mode() == 0) {   // one launch; lane pair = (party 0, party 1) of one element
-        // threads per CTA (PSML_MSB_TPB, multiple of 32, <= 256): smaller CTAs spread the chain's
-        // latency-bound lanes over more SMs
-        static int tpb = -1;
-        if (tpb < 0) {
-            const char *env = getenv("PSML_MSB_TPB");
-            const int v = env ? atoi(env) : EW_THREADS;
-            tpb = (v >= 32 && v <= 256 && v % 32 == 0) ? v : EW_THREADS;
-        }
+        const int tpb = EW_THREADS;
         const int64_t threads = what == 2 ? ((n / 2 + 7) / 8) * 32 : 2 * n;
         const int blocks = (int)((threads + tpb - 1) / tpb);
         cudaError_t e;

@@ -212,8 +212,8 @@ def test_explicit_mask_round_matches_fused_open():
 
 @pytest.mark.parametrize("env", [{"PSML_SEG": "simt"}, {"PSML_SEG": "tc"}, {"PSML_ROWS": "0", "PSML_CONV_GW": "generic"},
                                  {"PSML_DEAL_AFTER": "0", "PSML_DEAL_SPLIT": "0"},
-                                 {"PSML_DEAL_AFTER": "4", "PSML_DEAL_CTAS": "0", "PSML_DEAL_TILE": "64"}],
-                         ids=["seg_simt", "seg_tc", "rows_off_conv_gw_generic", "deal_at_fork_one_branch", "deal_late_full_grid_tile64"])
+                                 {"PSML_DEAL_AFTER": "4"}],
+                         ids=["seg_simt", "seg_tc", "rows_off_conv_gw_generic", "deal_at_fork_one_branch", "deal_late"])
 def test_seg_gemm_backends_match_oracle(env):
     """PSML_SEG=simt: every opened Beaver product of the training step on the CUDA-core
     two-segment GEMM; PSML_SEG=tc: every eligible one on the tcgen05 in-kernel-split GEMM
