@@ -306,6 +306,11 @@ typedef struct {
     int32_t weight_decay_shift; /* 0 = none; else W^m -= trunc(W^m, shift) every update (SVM:
                                    lambda.eta = 2^-16, R24)                        */
     int32_t rnn_steps;        /* RNN: sequence length T (1..254; call-id layers 1..T+1)       */
+    int32_t deal_role;        /* DESIGN.md R23: 0 = the dealer (dealer_seed = the dealer seed; every
+                                 stream), 1 / 2 = party 0 / 1 dealing for itself (dealer_seed =
+                                 that party's seed s_i = psml_dealer_party_seed(dealer seed, i));
+                                 the words it cannot derive come in the dealer's bundle
+                                 (psml_model_deal_bundle / psml_model_deal_party)              */
 } psml_model_desc;
 
 psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_model *out);
@@ -319,6 +324,22 @@ psml_status psml_model_set_master(psml_model model, int32_t layer, const void *c
                                   psml_stream stream);
 psml_status psml_model_get_master(psml_model model, int32_t layer, void *const Wm[2],
                                   psml_stream stream);
+/* Dealer key separation and compressed distribution (R23).  Party i's material streams
+ * are keyed by s_i = psml_dealer_party_seed(dealer_seed, i), so a party regenerates everything it
+ * can from s_i alone (party 0: all of its A2B-mode material) and receives only the derived words:
+ * party 1's Z_1 of every matrix / conv / Hadamard triplet, c_1 of every boolean AND triplet, r^A_1
+ * of every daBit; with the FSS comparison (compare = 1) a party's whole DCF material.
+ * psml_model_deal_bundle (a deal_role 0 model): deals `step_id` and gathers party `party`'s derived
+ * words into `bundle` (device, caller-owned; NULL = size query) -> *words.
+ * psml_model_deal_party (a deal_role 1 + party model): deals its own streams for `step_id` and
+ * scatters the bundle over the derived words; the pool is then identical to the dealer's for this
+ * party.  Both sides enumerate the words in the same order (items in plan order). */
+uint64_t psml_dealer_party_seed(uint64_t dealer_seed, int32_t party);
+psml_status psml_model_deal_bundle(psml_model model, uint32_t step_id, int32_t party, void *bundle, int64_t *words,
+                                   psml_stream stream);
+psml_status psml_model_deal_party(psml_model model, uint32_t step_id, int32_t party, const void *bundle,
+                                  int64_t words, psml_stream stream);
+
 /* Offline phase for one step: generate every triplet / MSB material the step's forward and
  * backward pass consumes, with call ids (pair_id, step_id, layer, op, slot) (R11).
  * infer_only = 1 generates only the forward material. */

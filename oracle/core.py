@@ -40,6 +40,10 @@ def lib():
         L.or_delta_csr_encode.restype = c_i64
         L.or_delta_csr_apply.argtypes = [c_i, c_i64, c_i64, ctypes.c_int32, vp, vp, vp, vp, vp]
         L.or_num_threads.restype = c_i
+        L.or_party_seed.argtypes = [c_u64, c_i]
+        L.or_party_seed.restype = c_u64
+        L.or_stream_seed.argtypes = [c_u64, c_u32]
+        L.or_stream_seed.restype = c_u64
         L.or_dcf_key_words.argtypes = [c_i]
         L.or_dcf_key_words.restype = c_i64
         L.or_dcf_gen.argtypes = [c_i, c_i, c_u64, c_u64, c_u64, c_u64, c_u64, c_u64, vp, vp]
@@ -85,6 +89,20 @@ def chacha20_block(key_words, counter, nonce_words):
     out = np.zeros(16, dtype=np.uint32)
     lib().or_chacha20_block(_p(k), counter, _p(n), _p(out))
     return out
+
+
+def party_seed(dealer_seed, party):
+    """s_i = PRG(dealer_seed, "KD", i)[0] (R23)."""
+    return lib().or_party_seed(dealer_seed, party)
+
+
+def stream_seed(dealer_seed, tag_value):
+    """The seed a dealer material stream is keyed by (R23): the owning party's, or the dealer's."""
+    return lib().or_stream_seed(dealer_seed, tag_value)
+
+
+def dealer_prg(l, dealer_seed, tag_value, call_id, n, offset=0):
+    return prg(l, stream_seed(dealer_seed, tag_value), tag_value, call_id, n, offset)
 
 
 def prg(l, seed, tag_value, call_id, n, offset=0):

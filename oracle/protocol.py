@@ -197,14 +197,14 @@ def conv_triplet(pair, step, op, B, transpose):
     rows = B * (g["H"] - g["k"] + 1) * (g["W"] - g["k"] + 1)
     kk = g["C"] * g["k"] * g["k"]
     vshape = (rows, g["Cout"]) if transpose else (kk, g["Cout"])
-    U0 = core.prg(L, DEALER_SEED, core.tag("U0"), cid, nin).reshape(B, -1)
-    U1 = core.prg(L, DEALER_SEED, core.tag("U1"), cid, nin).reshape(B, -1)
+    U0 = core.dealer_prg(L, DEALER_SEED, core.tag("U0"), cid, nin).reshape(B, -1)
+    U1 = core.dealer_prg(L, DEALER_SEED, core.tag("U1"), cid, nin).reshape(B, -1)
     nv = vshape[0] * vshape[1]
-    V0 = core.prg(L, DEALER_SEED, core.tag("V0"), cid, nv).reshape(vshape)
-    V1 = core.prg(L, DEALER_SEED, core.tag("V1"), cid, nv).reshape(vshape)
+    V0 = core.dealer_prg(L, DEALER_SEED, core.tag("V0"), cid, nv).reshape(vshape)
+    V1 = core.dealer_prg(L, DEALER_SEED, core.tag("V1"), cid, nv).reshape(vshape)
     Ucol = core.im2col(U0 + U1, g["C"], g["H"], g["W"], g["k"])
     Z = core.ring_matmul(np.ascontiguousarray(Ucol.T) if transpose else Ucol, V0 + V1)
-    Z0 = core.prg(L, DEALER_SEED, core.tag("Z0"), cid, Z.size).reshape(Z.shape)
+    Z0 = core.dealer_prg(L, DEALER_SEED, core.tag("Z0"), cid, Z.size).reshape(Z.shape)
     return (U0, U1), (V0, V1), (Z0, Z - Z0)
 
 

@@ -92,6 +92,32 @@ EXPORT void or_prg(int l, uint64_t seed, uint32_t tag, uint64_t id, uint64_t off
     }
 }
 
+/*
+ * Dealer key separation (R23).  The dealer (the paper's client) holds the
+ * dealer seed; party i holds only s_i = first word of PRG(dealer_seed, "KD", i) (R1 layout).  Every
+ * material stream a party can produce itself is keyed by that party's seed (U0, V0, Z0, a0, b0, c0,
+ * R0, RA, F0, FS, K0 -> s_0; U1, V1, a1, b1, R1, K1 -> s_1); streams only the dealer may know (the
+ * FSS input mask "FR") keep the dealer seed.  The derived words (Z_1, c_1, r^A_1, FSS correction
+ * words) need both seeds and are what the dealer ships (compressed distribution).
+ */
+EXPORT uint64_t or_party_seed(uint64_t dealer_seed, int party) {
+    uint64_t v;
+    or_prg(64, dealer_seed, 0x0000444Bu /* "KD" */, (uint64_t)party, 0, 1, &v);
+    return v;
+}
+
+EXPORT uint64_t or_stream_seed(uint64_t dealer_seed, uint32_t tag) {
+    int b0 = (int)(tag & 0xFF), b1 = (int)((tag >> 8) & 0xFF);
+    if (b1 == '1') return or_party_seed(dealer_seed, 1);
+    if (b1 == '0' || (b0 == 'R' && b1 == 'A') || (b0 == 'F' && b1 == 'S')) return or_party_seed(dealer_seed, 0);
+    return dealer_seed;
+}
+
+/* or_prg for a dealer material stream: keyed by or_stream_seed. */
+static void dprg(int l, uint64_t seed, uint32_t tag, uint64_t id, uint64_t offset, int64_t n, uint64_t *out) {
+    or_prg(l, or_stream_seed(seed, tag), tag, id, offset, n, out);
+}
+
 /* ------------------------------------------------------------------------------------------ */
 /* Fixed-point encoding (R3; SecureML fixed point, not in PAPER.md which is FP32,     */
 /* L248/L260): v = round_half_even(x * 2^f) mod 2^l;  decode = signed(v) / 2^f.               */
@@ -157,11 +183,11 @@ EXPORT void or_triplet_gen(int l, uint64_t seed, uint64_t call_id, int64_t M, in
                            uint64_t *U0, uint64_t *U1, uint64_t *V0, uint64_t *V1, uint64_t *Z0,
                            uint64_t *Z1) {
     uint64_t m = ring_mask(l);
-    or_prg(l, seed, TAG('U', '0', 0, 0), call_id, 0, M * K, U0);
-    or_prg(l, seed, TAG('U', '1', 0, 0), call_id, 0, M * K, U1);
-    or_prg(l, seed, TAG('V', '0', 0, 0), call_id, 0, K * N, V0);
-    or_prg(l, seed, TAG('V', '1', 0, 0), call_id, 0, K * N, V1);
-    or_prg(l, seed, TAG('Z', '0', 0, 0), call_id, 0, M * N, Z0);
+    dprg(l, seed, TAG('U', '0', 0, 0), call_id, 0, M * K, U0);
+    dprg(l, seed, TAG('U', '1', 0, 0), call_id, 0, M * K, U1);
+    dprg(l, seed, TAG('V', '0', 0, 0), call_id, 0, K * N, V0);
+    dprg(l, seed, TAG('V', '1', 0, 0), call_id, 0, K * N, V1);
+    dprg(l, seed, TAG('Z', '0', 0, 0), call_id, 0, M * N, Z0);
     uint64_t *U = malloc(sizeof(uint64_t) * M * K), *V = malloc(sizeof(uint64_t) * K * N);
     uint64_t *Z = malloc(sizeof(uint64_t) * M * N);
     for (int64_t i = 0; i < M * K; ++i) U[i] = (U0[i] + U1[i]) & m;   /* Eq. 3 */
@@ -175,11 +201,11 @@ EXPORT void or_hadamard_triplet_gen(int l, uint64_t seed, uint64_t call_id, int6
                                     uint64_t *U0, uint64_t *U1, uint64_t *V0, uint64_t *V1,
                                     uint64_t *Z0, uint64_t *Z1) {
     uint64_t m = ring_mask(l);
-    or_prg(l, seed, TAG('U', '0', 0, 0), call_id, 0, n, U0);
-    or_prg(l, seed, TAG('U', '1', 0, 0), call_id, 0, n, U1);
-    or_prg(l, seed, TAG('V', '0', 0, 0), call_id, 0, n, V0);
-    or_prg(l, seed, TAG('V', '1', 0, 0), call_id, 0, n, V1);
-    or_prg(l, seed, TAG('Z', '0', 0, 0), call_id, 0, n, Z0);
+    dprg(l, seed, TAG('U', '0', 0, 0), call_id, 0, n, U0);
+    dprg(l, seed, TAG('U', '1', 0, 0), call_id, 0, n, U1);
+    dprg(l, seed, TAG('V', '0', 0, 0), call_id, 0, n, V0);
+    dprg(l, seed, TAG('V', '1', 0, 0), call_id, 0, n, V1);
+    dprg(l, seed, TAG('Z', '0', 0, 0), call_id, 0, n, Z0);
     for (int64_t i = 0; i < n; ++i) Z1[i] = (((U0[i] + U1[i]) * (V0[i] + V1[i])) - Z0[i]) & m;
 }
 
@@ -289,11 +315,11 @@ EXPORT void or_msb_dealer(int l, uint64_t seed, uint64_t call_id, int64_t n, uin
     uint64_t *mat[2] = {mat0, mat1};
     for (int t = 0; t < 2 * L; ++t) {
         for (int i = 0; i < 2; ++i) {
-            or_prg(l, seed, TAG('a', '0' + i, t, 0), call_id, 0, n, mat[i] + ((int64_t)t * 3 + 0) * n);
-            or_prg(l, seed, TAG('b', '0' + i, t, 0), call_id, 0, n, mat[i] + ((int64_t)t * 3 + 1) * n);
+            dprg(l, seed, TAG('a', '0' + i, t, 0), call_id, 0, n, mat[i] + ((int64_t)t * 3 + 0) * n);
+            dprg(l, seed, TAG('b', '0' + i, t, 0), call_id, 0, n, mat[i] + ((int64_t)t * 3 + 1) * n);
         }
         uint64_t *c0 = mat0 + ((int64_t)t * 3 + 2) * n, *c1 = mat1 + ((int64_t)t * 3 + 2) * n;
-        or_prg(l, seed, TAG('c', '0', t, 0), call_id, 0, n, c0);
+        dprg(l, seed, TAG('c', '0', t, 0), call_id, 0, n, c0);
         for (int64_t e = 0; e < n; ++e) {
             uint64_t a = mat0[((int64_t)t * 3 + 0) * n + e] ^ mat1[((int64_t)t * 3 + 0) * n + e];
             uint64_t b = mat0[((int64_t)t * 3 + 1) * n + e] ^ mat1[((int64_t)t * 3 + 1) * n + e];
@@ -301,10 +327,10 @@ EXPORT void or_msb_dealer(int l, uint64_t seed, uint64_t call_id, int64_t n, uin
         }
     }
     int64_t off = (int64_t)2 * L * 3 * n;
-    or_prg(l, seed, TAG('R', '0', 0, 0), call_id, 0, n, mat0 + off);
-    or_prg(l, seed, TAG('R', '1', 0, 0), call_id, 0, n, mat1 + off);
+    dprg(l, seed, TAG('R', '0', 0, 0), call_id, 0, n, mat0 + off);
+    dprg(l, seed, TAG('R', '1', 0, 0), call_id, 0, n, mat1 + off);
     for (int64_t e = 0; e < n; ++e) { mat0[off + e] &= 1; mat1[off + e] &= 1; }
-    or_prg(l, seed, TAG('R', 'A', 0, 0), call_id, 0, n, mat0 + off + n);
+    dprg(l, seed, TAG('R', 'A', 0, 0), call_id, 0, n, mat0 + off + n);
     for (int64_t e = 0; e < n; ++e)
         mat1[off + n + e] = ((mat0[off + e] ^ mat1[off + e]) - mat0[off + n + e]) & m;
 }
@@ -550,11 +576,11 @@ EXPORT void or_fss_dealer(int l, uint64_t seed, uint64_t call_id, int64_t n, uin
     int64_t kw = or_dcf_key_words(nb);
     uint64_t *r = malloc(sizeof(uint64_t) * n), *r0 = malloc(sizeof(uint64_t) * n), *sa0 = malloc(sizeof(uint64_t) * n);
     uint64_t *K0 = malloc(sizeof(uint64_t) * 2 * n), *K1 = malloc(sizeof(uint64_t) * 2 * n);
-    or_prg(l, seed, 0x00005246u /* "FR" */, call_id, 0, n, r);
-    or_prg(l, seed, 0x00003046u /* "F0" */, call_id, 0, n, r0);
-    or_prg(l, seed, 0x00005346u /* "FS" */, call_id, 0, n, sa0);
-    or_prg(64, seed, 0x0000304Bu /* "K0" */, call_id, 0, 2 * n, K0);
-    or_prg(64, seed, 0x0000314Bu /* "K1" */, call_id, 0, 2 * n, K1);
+    dprg(l, seed, 0x00005246u /* "FR" */, call_id, 0, n, r);
+    dprg(l, seed, 0x00003046u /* "F0" */, call_id, 0, n, r0);
+    dprg(l, seed, 0x00005346u /* "FS" */, call_id, 0, n, sa0);
+    dprg(64, seed, 0x0000304Bu /* "K0" */, call_id, 0, 2 * n, K0);
+    dprg(64, seed, 0x0000314Bu /* "K1" */, call_id, 0, 2 * n, K1);
 #pragma omp parallel for schedule(static)
     for (int64_t e = 0; e < n; ++e) {
         uint64_t k0[4 * 64 + 3], k1[4 * 64 + 3];

@@ -132,6 +132,27 @@ __host__ __device__ inline PrgKey make_key(uint64_t seed, uint32_t tag, uint64_t
     return k;
 }
 
+// Dealer key separation (R23): each material stream is keyed by the seed of the party
+// that can produce it alone -- s_0 for U0 V0 Z0 a0 b0 c0 R0 RA F0 FS K0, s_1 for U1 V1 a1 b1 R1 K1 --
+// or by the dealer seed (the FSS input mask "FR").  s_i = PRG(dealer seed, "KD", i)[0].  A party that
+// deals for itself alone holds only its s_i (the other entries are 0 and their streams are junk,
+// overwritten by the dealer's bundle of derived words).
+struct DealSeeds {
+    uint64_t d, s0, s1;
+};
+__host__ __device__ inline uint64_t seed_for(const DealSeeds &S, uint32_t tag) {
+    const uint32_t b0 = tag & 0xFF, b1 = (tag >> 8) & 0xFF;
+    if (b1 == '1') return S.s1;
+    if (b1 == '0' || (b0 == 'R' && b1 == 'A') || (b0 == 'F' && b1 == 'S')) return S.s0;
+    return S.d;
+}
+__host__ __device__ inline PrgKey dkey(const DealSeeds &S, uint32_t tag, uint64_t call_id,
+                                       const uint32_t *step = nullptr) {
+    return make_key(seed_for(S, tag), tag, call_id, step);
+}
+// Host: the seeds of a full dealer (engine.cu).
+DealSeeds dealer_seeds(uint64_t dealer_seed);
+
 // Resolve the step field from device memory (call id = pair|step|layer|op|slot, R11),
 // so a captured graph replays with a new step number without re-instantiation.
 __device__ __forceinline__ PrgKey live_key(PrgKey k) {

@@ -54,18 +54,18 @@ __device__ __forceinline__ void deal_block(const PrgKey &k, uint32_t b, uint64_t
 // Streams 2..4 of a Hadamard (U0 U1 V0 V1 Z0 -> Z1 = (U0+U1)(V0+V1) - Z0) or boolean AND
 // (a0 a1 b0 b1 c0 -> c1 = ((a0^a1)&(b0^b1))^c0) job; x holds stream 0, v stream 1.
 template <bool HAD>
-__device__ __forceinline__ void deal_tail(const PrgJob &J, uint64_t seed, uint64_t cid, uint32_t b, int64_t e0, int64_t n,
+__device__ __forceinline__ void deal_tail(const PrgJob &J, const DealSeeds &S, uint64_t cid, uint32_t b, int64_t e0, int64_t n,
                                           uint64_t x[8], uint64_t v[8]) {
     uint64_t y[8];
 #pragma unroll
     for (int j = 0; j < 8; ++j) x[j] = HAD ? x[j] + v[j] : x[j] ^ v[j];
-    deal_block(make_key(seed, J.tag[2], cid), b, y);
+    deal_block(dkey(S, J.tag[2], cid), b, y);
     deal_store8(J.out[2], e0, n, y);
-    deal_block(make_key(seed, J.tag[3], cid), b, v);
+    deal_block(dkey(S, J.tag[3], cid), b, v);
     deal_store8(J.out[3], e0, n, v);
 #pragma unroll
     for (int j = 0; j < 8; ++j) x[j] = HAD ? x[j] * (y[j] + v[j]) : x[j] & (y[j] ^ v[j]);
-    deal_block(make_key(seed, J.tag[4], cid), b, v);
+    deal_block(dkey(S, J.tag[4], cid), b, v);
     deal_store8(J.out[4], e0, n, v);
 #pragma unroll
     for (int j = 0; j < 8; ++j) x[j] = HAD ? x[j] - v[j] : x[j] ^ v[j];
@@ -77,7 +77,7 @@ __device__ __forceinline__ void deal_tail(const PrgJob &J, uint64_t seed, uint64
 // the bounded PRG grid (PSML_DEAL_CTAS per SM) leaves part of each SM's register file to the
 // online phase it runs beside.
 __global__ void __launch_bounds__(128, PSML_DEAL_MINB) deal_prg_kernel(const PrgJob *__restrict__ jobs, int njobs, int64_t blk_first,
-                                                           int64_t total_blk, uint64_t seed, const uint32_t *step) {
+                                                           int64_t total_blk, const DealSeeds S, const uint32_t *step) {
     for (int64_t g = blk_first + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; g < total_blk;
          g += (int64_t)gridDim.x * blockDim.x) {
         int lo = 0, hi = njobs - 1;   // last job with blk_begin <= g
@@ -90,16 +90,16 @@ __global__ void __launch_bounds__(128, PSML_DEAL_MINB) deal_prg_kernel(const Prg
         const uint64_t cid = cid_with_step(J.cid, step);
         const int kind = J.kind;
         uint64_t v[8], x[8], y[8];
-        deal_block(make_key(seed, J.tag[0], cid), (uint32_t)b, v);
+        deal_block(dkey(S, J.tag[0], cid), (uint32_t)b, v);
         if (kind == PJ_DABIT) {
 #pragma unroll
             for (int j = 0; j < 8; ++j) { x[j] = v[j] & 1; }
             deal_store8(J.out[0], e0, n, x);
-            deal_block(make_key(seed, J.tag[1], cid), (uint32_t)b, v);
+            deal_block(dkey(S, J.tag[1], cid), (uint32_t)b, v);
 #pragma unroll
             for (int j = 0; j < 8; ++j) { v[j] &= 1; x[j] ^= v[j]; }
             deal_store8(J.out[1], e0, n, v);
-            deal_block(make_key(seed, J.tag[2], cid), (uint32_t)b, v);   // r^A_0
+            deal_block(dkey(S, J.tag[2], cid), (uint32_t)b, v);   // r^A_0
             deal_store8(J.out[2], e0, n, v);
 #pragma unroll
             for (int j = 0; j < 8; ++j) x[j] -= v[j];                    // r^A_1 = (r0 ^ r1) - r^A_0
@@ -110,11 +110,11 @@ __global__ void __launch_bounds__(128, PSML_DEAL_MINB) deal_prg_kernel(const Prg
         if (kind == PJ_SINGLE) continue;
 #pragma unroll
         for (int j = 0; j < 8; ++j) x[j] = v[j];
-        deal_block(make_key(seed, J.tag[1], cid), (uint32_t)b, v);
+        deal_block(dkey(S, J.tag[1], cid), (uint32_t)b, v);
         deal_store8(J.out[1], e0, n, v);
         if (kind == PJ_PAIR) continue;
-        if (kind == PJ_HAD) deal_tail<true>(J, seed, cid, (uint32_t)b, e0, n, x, v);
-        else deal_tail<false>(J, seed, cid, (uint32_t)b, e0, n, x, v);
+        if (kind == PJ_HAD) deal_tail<true>(J, S, cid, (uint32_t)b, e0, n, x, v);
+        else deal_tail<false>(J, S, cid, (uint32_t)b, e0, n, x, v);
     }
 }
 

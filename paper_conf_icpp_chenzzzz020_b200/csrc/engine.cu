@@ -168,6 +168,43 @@ psml_status psml_bench_mac_peak(int32_t l, double *ring_macs_per_s) {
     return PSML_OK;
 }
 
+namespace psml {
+// Host ChaCha20 block (RFC 8439 Sec. 2.3), used only to derive the parties' dealer seeds.
+static void host_chacha20(const uint32_t key[8], uint32_t counter, const uint32_t nonce[3], uint32_t out[16]) {
+    auto rl = [](uint32_t v, int c) { return (v << c) | (v >> (32 - c)); };
+    uint32_t st[16] = {0x61707865u, 0x3320646eu, 0x79622d32u, 0x6b206574u, key[0], key[1], key[2], key[3],
+                       key[4],      key[5],      key[6],      key[7],      counter, nonce[0], nonce[1], nonce[2]};
+    uint32_t x[16];
+    for (int i = 0; i < 16; ++i) x[i] = st[i];
+    auto qr = [&](int a, int b, int c, int d) {
+        x[a] += x[b]; x[d] ^= x[a]; x[d] = rl(x[d], 16);
+        x[c] += x[d]; x[b] ^= x[c]; x[b] = rl(x[b], 12);
+        x[a] += x[b]; x[d] ^= x[a]; x[d] = rl(x[d], 8);
+        x[c] += x[d]; x[b] ^= x[c]; x[b] = rl(x[b], 7);
+    };
+    for (int r = 0; r < 10; ++r) {
+        qr(0, 4, 8, 12); qr(1, 5, 9, 13); qr(2, 6, 10, 14); qr(3, 7, 11, 15);
+        qr(0, 5, 10, 15); qr(1, 6, 11, 12); qr(2, 7, 8, 13); qr(3, 4, 9, 14);
+    }
+    for (int i = 0; i < 16; ++i) out[i] = x[i] + st[i];
+}
+
+// s_i = element 0 of the PRG stream (dealer seed, "KD", call id i)  (R1, R23)
+static uint64_t party_seed(uint64_t dealer_seed, int party) {
+    const uint32_t key[8] = {(uint32_t)dealer_seed, (uint32_t)(dealer_seed >> 32), 0, 0, 0, 0, 0, 0};
+    const uint32_t nonce[3] = {0x0000444Bu /* "KD" */, (uint32_t)party, 0};
+    uint32_t w[16];
+    host_chacha20(key, 0, nonce, w);
+    return ((uint64_t)w[1] << 32) | w[0];
+}
+
+DealSeeds dealer_seeds(uint64_t dealer_seed) { return DealSeeds{dealer_seed, party_seed(dealer_seed, 0), party_seed(dealer_seed, 1)}; }
+}  // namespace psml
+
+uint64_t psml_dealer_party_seed(uint64_t dealer_seed, int32_t party) {
+    return (party == 0 || party == 1) ? party_seed(dealer_seed, party) : 0;
+}
+
 psml_status psml_device_info(int32_t *sm_count, int32_t *cc_major, int32_t *cc_minor) {
     int dev = 0, n = 0;
     if (cudaGetDeviceCount(&n) != cudaSuccess || n == 0) {
@@ -238,10 +275,11 @@ psml_status psml_secure_matmul_party(psml_ctx ctx, const void *A_i, const void *
     if (c->party < 0 || !c->xport) return fail(PSML_ERR_STATE, "not a per-party context (psml_ctx_create_party)");
     if (M <= 0 || K <= 0 || N <= 0) return fail(PSML_ERR_SHAPE, "M, K, N must be positive");
     const size_t w = c->ring.l / 8;
-    PSML_TRY(c->ensure_msg(w * 2 * (size_t)(M * K + K * N) + 512));
+    auto up = [](size_t x) { return (x + 255) & ~(size_t)255; };   // 16-byte aligned sub-buffers
+    const size_t eb = up(w * M * K), fb = up(w * K * N);
+    PSML_TRY(c->ensure_msg(2 * (eb + fb)));
     uint8_t *b = (uint8_t *)c->msg;
-    void *Es = b, *Fs = b + w * M * K;
-    void *Er = b + w * (M * K + K * N), *Fr = b + w * (2 * M * K + K * N);
+    void *Es = b, *Fs = b + eb, *Er = b + eb + fb, *Fr = b + 2 * eb + fb;
     // round 1 (Eq. 4), the exchange of E_i and F_i (Eq. 5) through the pair transport, round 2
     PSML_TRY(psml_beaver_mask(ctx, c->party, A_i, B_i, U_i, V_i, M, K, N, flags, Es, Fs, stream));
     const void *snd[2] = {Es, Fs};
@@ -394,13 +432,14 @@ psml_status psml_reconstruct(psml_ring ring, const void *x0, const void *x1, int
 template <typename T>
 static psml_status triplet_gen_t(Ctx *c, uint64_t seed, uint64_t cid, int64_t M, int64_t K, int64_t N,
                                  void *const U[2], void *const V[2], void *const Z[2], cudaStream_t s) {
-    dealer_pair_kernel<T><<<grid_for(M * K / 8 + 1, 256), 256, 0, s>>>(make_key(seed, TAG_U0, cid), make_key(seed, TAG_U1, cid), M * K,
+    const DealSeeds S = dealer_seeds(seed);
+    dealer_pair_kernel<T><<<grid_for(M * K / 8 + 1, 256), 256, 0, s>>>(dkey(S, TAG_U0, cid), dkey(S, TAG_U1, cid), M * K,
                                                                        (T *)U[0], (T *)U[1], nullptr);
     PSML_LAUNCH_CHECK();
-    dealer_pair_kernel<T><<<grid_for(K * N / 8 + 1, 256), 256, 0, s>>>(make_key(seed, TAG_V0, cid), make_key(seed, TAG_V1, cid), K * N,
+    dealer_pair_kernel<T><<<grid_for(K * N / 8 + 1, 256), 256, 0, s>>>(dkey(S, TAG_V0, cid), dkey(S, TAG_V1, cid), K * N,
                                                                        (T *)V[0], (T *)V[1], nullptr);
     PSML_LAUNCH_CHECK();
-    prg_kernel<T, 0><<<grid_for(M * N / 8 + 2, 256), 256, 0, s>>>(make_key(seed, TAG_Z0, cid), 0, M * N, (T *)Z[0],
+    prg_kernel<T, 0><<<grid_for(M * N / 8 + 2, 256), 256, 0, s>>>(dkey(S, TAG_Z0, cid), 0, M * N, (T *)Z[0],
                                                                   nullptr, nullptr);
     PSML_LAUNCH_CHECK();
     // Z = (U0+U1)(V0+V1) on the tensor cores where it pays, else the CUDA-core ring GEMM
@@ -441,8 +480,8 @@ psml_status psml_hadamard_triplet_gen(psml_ring ring, uint64_t seed, uint64_t ca
     PSML_TRY(check_ptrs({U[0], U[1], V[0], V[1], Z[0], Z[1]}));
     cudaStream_t s = (cudaStream_t)stream;
     if (ring.l == 64)
-        return hadamard_triplet_launch<uint64_t>(seed, call_id, n, U, V, Z, s);
-    return hadamard_triplet_launch<uint32_t>(seed, call_id, n, U, V, Z, s);
+        return hadamard_triplet_launch<uint64_t>(dealer_seeds(seed), call_id, n, U, V, Z, s);
+    return hadamard_triplet_launch<uint32_t>(dealer_seeds(seed), call_id, n, U, V, Z, s);
 }
 
 int64_t psml_msb_material_words(psml_ring ring, int64_t n) {
@@ -458,8 +497,8 @@ psml_status psml_msb_dealer(psml_ring ring, uint64_t seed, uint64_t call_id, int
     if (!mat) return fail(PSML_ERR_INVALID, "null pair array");
     PSML_TRY(check_ptrs({mat[0], mat[1]}));
     cudaStream_t s = (cudaStream_t)stream;
-    if (ring.l == 64) return msb_dealer_launch<uint64_t>(seed, call_id, n, mat, s);
-    return msb_dealer_launch<uint32_t>(seed, call_id, n, mat, s);
+    if (ring.l == 64) return msb_dealer_launch<uint64_t>(dealer_seeds(seed), call_id, n, mat, s);
+    return msb_dealer_launch<uint32_t>(dealer_seeds(seed), call_id, n, mat, s);
 }
 
 // ------------------------------------------------------------------------------------------------
@@ -726,7 +765,7 @@ psml_status psml_fss_dealer(psml_ring ring, uint64_t seed, uint64_t call_id, int
     PSML_TRY(check_ptrs({mat[0], mat[1]}));
     cudaStream_t s = (cudaStream_t)stream;
     ProfScope prof(PROF_DEALER, s, 2.0 * FSS_BITS * (double)n);
-    return fss_dealer_launch(seed, call_id, n, (uint64_t *)mat[0], (uint64_t *)mat[1], s);
+    return fss_dealer_launch(dealer_seeds(seed), call_id, n, (uint64_t *)mat[0], (uint64_t *)mat[1], s);
 }
 
 static psml_status fss_drelu_pair(const void *const x[2], int64_t n, const void *const mat[2], uint64_t *const d[2],

@@ -40,24 +40,24 @@ struct Ctx {
 // launch helpers (templates, used by engine.cu and model.cu)
 // ------------------------------------------------------------------------------------------------
 template <typename T>
-psml_status hadamard_triplet_launch(uint64_t seed, uint64_t cid, int64_t n, void *const U[2], void *const V[2],
+psml_status hadamard_triplet_launch(const DealSeeds &S, uint64_t cid, int64_t n, void *const U[2], void *const V[2],
                                     void *const Z[2], cudaStream_t s, const uint32_t *step = nullptr) {
     Pair<T> u{{(T *)U[0], (T *)U[1]}}, v{{(T *)V[0], (T *)V[1]}}, z{{(T *)Z[0], (T *)Z[1]}};
     const int64_t nblk = (n + PerBlock<T>::value - 1) / PerBlock<T>::value;
     hadamard_triplet_kernel<T><<<grid_for(nblk, 128, 148 * 32), 128, 0, s>>>(
-        make_key(seed, TAG_U0, cid, step), make_key(seed, TAG_U1, cid, step), make_key(seed, TAG_V0, cid, step),
-        make_key(seed, TAG_V1, cid, step), make_key(seed, TAG_Z0, cid, step), n, u, v, z);
+        dkey(S, TAG_U0, cid, step), dkey(S, TAG_U1, cid, step), dkey(S, TAG_V0, cid, step),
+        dkey(S, TAG_V1, cid, step), dkey(S, TAG_Z0, cid, step), n, u, v, z);
     PSML_LAUNCH_CHECK();
     return PSML_OK;
 }
 
 template <typename T>
-psml_status msb_dealer_launch(uint64_t seed, uint64_t cid, int64_t n, void *const mat[2], cudaStream_t s,
+psml_status msb_dealer_launch(const DealSeeds &S, uint64_t cid, int64_t n, void *const mat[2], cudaStream_t s,
                               const uint32_t *step = nullptr) {
     const int L = ilog2_int(8 * (int)sizeof(T));
     const int64_t nblk = (n + PerBlock<T>::value - 1) / PerBlock<T>::value;
     dim3 grid((unsigned)grid_for(nblk, 128, 148 * 8), (unsigned)(2 * L + 1));
-    msb_dealer_kernel<T><<<grid, 128, 0, s>>>(seed, cid, n, L, (T *)mat[0], (T *)mat[1], step);
+    msb_dealer_kernel<T><<<grid, 128, 0, s>>>(S, cid, n, L, (T *)mat[0], (T *)mat[1], step);
     PSML_LAUNCH_CHECK();
     return PSML_OK;
 }

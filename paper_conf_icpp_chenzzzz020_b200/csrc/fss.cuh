@@ -185,12 +185,12 @@ static __global__ void __launch_bounds__(256) eq9_combine_kernel(CPair<uint64_t>
 }
 
 // Dealer launch with keys whose step field may live in device memory (CUDA graphs).
-static inline psml_status fss_dealer_launch(uint64_t seed, uint64_t cid, int64_t n, uint64_t *m0, uint64_t *m1,
+static inline psml_status fss_dealer_launch(const DealSeeds &S, uint64_t cid, int64_t n, uint64_t *m0, uint64_t *m1,
                                             cudaStream_t s, const uint32_t *step = nullptr) {
     if (n <= 0) return PSML_OK;
     fss_dealer_kernel<<<grid_for(n, 128, 148 * 16), 128, 0, s>>>(
-        make_key(seed, TAG_FR, cid, step), make_key(seed, TAG_F0, cid, step), make_key(seed, TAG_FS, cid, step),
-        make_key(seed, TAG_K0, cid, step), make_key(seed, TAG_K1, cid, step), n, m0, m1);
+        dkey(S, TAG_FR, cid, step), dkey(S, TAG_F0, cid, step), dkey(S, TAG_FS, cid, step),
+        dkey(S, TAG_K0, cid, step), dkey(S, TAG_K1, cid, step), n, m0, m1);
     PSML_LAUNCH_CHECK();
     return PSML_OK;
 }

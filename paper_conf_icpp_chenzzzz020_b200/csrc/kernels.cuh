@@ -176,7 +176,7 @@ __global__ void hadamard_triplet_kernel(PrgKey ku0, PrgKey ku1, PrgKey kv0, PrgK
 
 // MSB material: blockIdx.y = AND index t (0 .. 2L-1) or 2L for the daBit.
 template <typename T>
-__global__ void msb_dealer_kernel(uint64_t seed, uint64_t call_id, int64_t n, int L, T *__restrict__ m0,
+__global__ void msb_dealer_kernel(const DealSeeds S, uint64_t call_id, int64_t n, int L, T *__restrict__ m0,
                                   T *__restrict__ m1, const uint32_t *step) {
     constexpr int PB = PerBlock<T>::value;
     if (step) {
@@ -188,11 +188,11 @@ __global__ void msb_dealer_kernel(uint64_t seed, uint64_t call_id, int64_t n, in
     for (int64_t b = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; b < nblk; b += (int64_t)gridDim.x * blockDim.x) {
         if (t < 2 * L) {
             uint32_t wa0[16], wa1[16], wb0[16], wb1[16], wc0[16];
-            chacha20_block(make_key(seed, tag4('a', '0', t), call_id), (uint32_t)b, wa0);
-            chacha20_block(make_key(seed, tag4('a', '1', t), call_id), (uint32_t)b, wa1);
-            chacha20_block(make_key(seed, tag4('b', '0', t), call_id), (uint32_t)b, wb0);
-            chacha20_block(make_key(seed, tag4('b', '1', t), call_id), (uint32_t)b, wb1);
-            chacha20_block(make_key(seed, tag4('c', '0', t), call_id), (uint32_t)b, wc0);
+            chacha20_block(dkey(S, tag4('a', '0', t), call_id), (uint32_t)b, wa0);
+            chacha20_block(dkey(S, tag4('a', '1', t), call_id), (uint32_t)b, wa1);
+            chacha20_block(dkey(S, tag4('b', '0', t), call_id), (uint32_t)b, wb0);
+            chacha20_block(dkey(S, tag4('b', '1', t), call_id), (uint32_t)b, wb1);
+            chacha20_block(dkey(S, tag4('c', '0', t), call_id), (uint32_t)b, wc0);
             T *base0 = m0 + (int64_t)t * 3 * n, *base1 = m1 + (int64_t)t * 3 * n;
 #pragma unroll
             for (int j = 0; j < PB; ++j) {
@@ -205,9 +205,9 @@ __global__ void msb_dealer_kernel(uint64_t seed, uint64_t call_id, int64_t n, in
             }
         } else {
             uint32_t w0[16], w1[16], wa[16];
-            chacha20_block(make_key(seed, TAG_R0, call_id), (uint32_t)b, w0);
-            chacha20_block(make_key(seed, TAG_R1, call_id), (uint32_t)b, w1);
-            chacha20_block(make_key(seed, TAG_RA, call_id), (uint32_t)b, wa);
+            chacha20_block(dkey(S, TAG_R0, call_id), (uint32_t)b, w0);
+            chacha20_block(dkey(S, TAG_R1, call_id), (uint32_t)b, w1);
+            chacha20_block(dkey(S, TAG_RA, call_id), (uint32_t)b, wa);
             const int64_t off = (int64_t)2 * L * 3 * n;
 #pragma unroll
             for (int j = 0; j < PB; ++j) {

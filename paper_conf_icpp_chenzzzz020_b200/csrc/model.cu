@@ -156,6 +156,7 @@ struct psml_model_s {
     // split deployment capture (psml_party_capture_step): the party, its pair transport and its
     // data-parallel communicator; cap_party < 0 = the co-resident engine
     int cap_party = -1;
+    psml::DealSeeds seeds{};           // dealer key separation (R23), from dealer_seed and deal_role
     // RNN (R25): per time step inputs A_t = [x_t | h_{t-1}], states h_t, DReLU_t, and the
     // per-step weight-gradient product before it is added into the layer-0 gradient
     psml::Buf rnnA, rnnH, rnnD, rnnG;
@@ -363,17 +364,17 @@ static int64_t dws_need(psml_model_s *m) {
 // ------------------------------------------------------------------------------------------------
 // PRG part of a matrix / conv triplet: U_0, U_1 (n_u), V_0, V_1 (K x N), Z_0 (M x N)
 static psml_status deal_prg(psml_model_s *m, DealItem &it, uint64_t cid, cudaStream_t s) {
-    const uint64_t seed = m->d.dealer_seed;
+    const DealSeeds &S = m->seeds;
     ProfScope prof(PROF_DEALER, s, (double)sizeof(T) * (2 * it.U.n + 2 * it.V.n + it.Z.n));
     dealer_pair_kernel<T><<<grid_for(it.U.n / 8 + 1, 256), 256, 0, s>>>(
-        make_key(seed, TAG_U0, cid, m->step_dev), make_key(seed, TAG_U1, cid, m->step_dev), it.U.n, it.U.p[0],
+        dkey(S, TAG_U0, cid, m->step_dev), dkey(S, TAG_U1, cid, m->step_dev), it.U.n, it.U.p[0],
         it.U.p[1], nullptr);
     PSML_LAUNCH_CHECK();
     dealer_pair_kernel<T><<<grid_for(it.V.n / 8 + 1, 256), 256, 0, s>>>(
-        make_key(seed, TAG_V0, cid, m->step_dev), make_key(seed, TAG_V1, cid, m->step_dev), it.V.n, it.V.p[0],
+        dkey(S, TAG_V0, cid, m->step_dev), dkey(S, TAG_V1, cid, m->step_dev), it.V.n, it.V.p[0],
         it.V.p[1], nullptr);
     PSML_LAUNCH_CHECK();
-    prg_kernel<T, 0><<<grid_for(it.Z.n / 8 + 2, 256), 256, 0, s>>>(make_key(seed, TAG_Z0, cid, m->step_dev), 0, it.Z.n,
+    prg_kernel<T, 0><<<grid_for(it.Z.n / 8 + 2, 256), 256, 0, s>>>(dkey(S, TAG_Z0, cid, m->step_dev), 0, it.Z.n,
                                                                      it.Z.p[0], nullptr, nullptr);
     PSML_LAUNCH_CHECK();
     return PSML_OK;
@@ -410,16 +411,16 @@ static psml_status deal_item(psml_model_s *m, DealItem &it, uint32_t step, cudaS
     case IT_HAD: {
         ProfScope prof(PROF_DEALER, s, (double)sizeof(T) * 6 * it.n);
         void *U[2] = {it.U.p[0], it.U.p[1]}, *V[2] = {it.V.p[0], it.V.p[1]}, *Z[2] = {it.Z.p[0], it.Z.p[1]};
-        return hadamard_triplet_launch<T>(seed, cid, it.n, U, V, Z, s, m->step_dev);
+        return hadamard_triplet_launch<T>(m->seeds, cid, it.n, U, V, Z, s, m->step_dev);
     }
     case IT_MSB: {
         ProfScope prof(PROF_DEALER, s, (double)sizeof(T) * 2 * it.mat.n);
         void *mt[2] = {it.mat.p[0], it.mat.p[1]};
-        return msb_dealer_launch<T>(seed, cid, it.n, mt, s, m->step_dev);
+        return msb_dealer_launch<T>(m->seeds, cid, it.n, mt, s, m->step_dev);
     }
     case IT_FSS: {
         ProfScope prof(PROF_DEALER, s, 2.0 * FSS_BITS * (double)it.n);
-        return fss_dealer_launch(seed, cid, it.n, it.mat.p[0], it.mat.p[1], s, m->step_dev);
+        return fss_dealer_launch(m->seeds, cid, it.n, it.mat.p[0], it.mat.p[1], s, m->step_dev);
     }
     }
     return PSML_OK;
@@ -550,7 +551,7 @@ static psml_status deal_prg_launch(psml_model_s *m, const DealPlan &P, int j0, i
     // overlaps nothing but the update: it takes the whole GPU
     const int64_t grid = (per_sm > 0 && !m->deal_alone) ? std::min<int64_t>(full, (int64_t)per_sm * m->ctx->sm_count)
                                                         : full;
-    deal_prg_kernel<<<(unsigned)grid, 128, 0, s>>>(P.prg + j0, j1 - j0, b0, b1, m->d.dealer_seed, m->step_dev);
+    deal_prg_kernel<<<(unsigned)grid, 128, 0, s>>>(P.prg + j0, j1 - j0, b0, b1, m->seeds, m->step_dev);
     PSML_LAUNCH_CHECK();
     return PSML_OK;
 }
@@ -1409,6 +1410,10 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
     std::unique_ptr<psml_model_s> m(new psml_model_s());
     m->ctx = c;
     m->d = *desc;
+    if (desc->deal_role < 0 || desc->deal_role > 2) return fail(PSML_ERR_INVALID, "deal_role must be 0, 1 or 2");
+    if (desc->deal_role == 0) m->seeds = dealer_seeds(desc->dealer_seed);           // the dealer: all streams
+    else if (desc->deal_role == 1) m->seeds = DealSeeds{0, desc->dealer_seed, 0};   // party 0 holds s_0 only
+    else m->seeds = DealSeeds{0, 0, desc->dealer_seed};                             // party 1 holds s_1 only
     m->B = desc->batch;
     switch (desc->kind) {
     case PSML_LINREG:
@@ -1612,6 +1617,73 @@ psml_status psml_model_deal(psml_model m, uint32_t step_id, int32_t infer_only, 
     PSML_TRY(deal_pool(m, pool, step_id, infer_only != 0, s));
     m->dealt_step[pool] = step_id;
     m->dealt_full[pool] = !infer_only;
+    return PSML_OK;
+}
+
+// Words of party `party`'s material that its own seed cannot produce, in plan order (R23).
+static std::vector<std::pair<T *, int64_t>> derived_regions(psml_model_s *m, int pool, int party) {
+    std::vector<std::pair<T *, int64_t>> r;
+    const int L = 6;   // log2(64): 2L AND triplets per MSB element
+    for (auto &it : m->items[pool]) {
+        switch (it.kind) {
+        case IT_MATRIX:
+        case IT_CONV_FWD:
+        case IT_CONV_GW:
+        case IT_HAD:
+            if (party == 1) r.push_back({it.Z.p[1], it.Z.n});                 // Z_1 = U V - Z_0
+            break;
+        case IT_MSB:
+            if (party == 1) {
+                for (int t = 0; t < 2 * L; ++t) r.push_back({it.mat.p[1] + (3 * (int64_t)t + 2) * it.n, it.n});   // c_1
+                r.push_back({it.mat.p[1] + (6 * (int64_t)L + 1) * it.n, it.n});                                 // r^A_1
+            }
+            break;
+        case IT_FSS:
+            r.push_back({it.mat.p[party], (int64_t)FSS_WORDS * it.n});        // DCF keys need both seeds
+            break;
+        }
+    }
+    return r;
+}
+
+psml_status psml_model_deal_bundle(psml_model m, uint32_t step_id, int32_t party, void *bundle, int64_t *words,
+                                   psml_stream stream) {
+    if (!m || !words) return fail(PSML_ERR_INVALID, "null argument");
+    if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
+    if (m->d.deal_role != 0) return fail(PSML_ERR_STATE, "only the dealer (deal_role 0) writes bundles");
+    const int pool = (int)(step_id & 1);
+    int64_t tot = 0;
+    for (auto &r : derived_regions(m, pool, party)) tot += r.second;
+    *words = tot;
+    if (!bundle) return PSML_OK;
+    PSML_TRY(check_ptrs({bundle}));
+    PSML_TRY(psml_model_deal(m, step_id, 0, stream));
+    T *out = (T *)bundle;
+    for (auto &r : derived_regions(m, pool, party)) {
+        PSML_CUDA_TRY(cudaMemcpyAsync(out, r.first, sizeof(T) * r.second, cudaMemcpyDeviceToDevice, (cudaStream_t)stream));
+        out += r.second;
+    }
+    m->dealt_step[pool] = -1;   // the dealer's own copy is not a party's pool
+    return PSML_OK;
+}
+
+psml_status psml_model_deal_party(psml_model m, uint32_t step_id, int32_t party, const void *bundle, int64_t words,
+                                  psml_stream stream) {
+    if (!m) return fail(PSML_ERR_INVALID, "model is null");
+    if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
+    if (m->d.deal_role != party + 1) return fail(PSML_ERR_STATE, "model deal_role is not this party's");
+    const int pool = (int)(step_id & 1);
+    int64_t tot = 0;
+    for (auto &r : derived_regions(m, pool, party)) tot += r.second;
+    if (words != tot) return fail(PSML_ERR_SHAPE, "bundle size does not match this model's derived words");
+    if (tot && !bundle) return fail(PSML_ERR_INVALID, "bundle is null");
+    PSML_TRY(check_ptrs({bundle}));
+    PSML_TRY(psml_model_deal(m, step_id, 0, stream));   // this party's own streams (the rest is junk)
+    const T *in = (const T *)bundle;
+    for (auto &r : derived_regions(m, pool, party)) {
+        PSML_CUDA_TRY(cudaMemcpyAsync(r.first, in, sizeof(T) * r.second, cudaMemcpyDeviceToDevice, (cudaStream_t)stream));
+        in += r.second;
+    }
     return PSML_OK;
 }
 

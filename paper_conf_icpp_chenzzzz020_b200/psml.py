@@ -45,7 +45,7 @@ class ModelDesc(ctypes.Structure):
                 ("pair_id", u32), ("cnn_c", i32), ("cnn_h", i32), ("cnn_w", i32), ("cnn_k", i32),
                 ("cnn_cout", i32), ("cnn_hidden", i32), ("cnn_classes", i32),
                 ("fwd_frac_bits", i32 * 8), ("compare", i32), ("weight_decay_shift", i32),
-                ("rnn_steps", i32)]
+                ("rnn_steps", i32), ("deal_role", i32)]
 
 
 # psml_exchange_fn (include/psml.h): (user, n, send[], recv[], bytes[], stream) -> 0 on success
@@ -119,6 +119,9 @@ _SIGS = {
     "psml_party_train_step": (i32, [vp, i32, vp, vp, vp, vp, u32, vp]),
     "psml_ctx_create_party": (i32, [Ring, i32, i32, vp, vp, vp]),
     "psml_secure_matmul_party": (i32, [vp, vp, vp, vp, vp, vp, i64, i64, i64, i32, i32, vp, vp]),
+    "psml_dealer_party_seed": (u64, [u64, i32]),
+    "psml_model_deal_bundle": (i32, [vp, u32, i32, vp, vp, vp]),
+    "psml_model_deal_party": (i32, [vp, u32, i32, vp, i64, vp]),
     "psml_fss_material_words": (i64, [Ring, i64]),
     "psml_fss_dealer": (i32, [Ring, u64, u64, i64, P2, vp]),
     "psml_secure_drelu_fss": (i32, [vp, P2, i64, P2, P2, vp, vp]),
@@ -224,6 +227,11 @@ def bench_mac_peak(l=64):
     v = ctypes.c_double()
     _call("psml_bench_mac_peak", l, ctypes.byref(v))
     return v.value
+
+
+def dealer_party_seed(dealer_seed, party):
+    """s_i = PRG(dealer seed, "KD", i)[0]: the only dealer secret party i holds (R23)."""
+    return lib().psml_dealer_party_seed(dealer_seed, party)
 
 
 def prof_enable(cls):
@@ -532,7 +540,7 @@ class Model:
 
     def __init__(self, ctx, kind, dims=None, batch=128, lr_shift=14, master_frac_bits=27,
                  dealer_seed=0x50534D4C + 2, pair_id=0, cnn=(3, 32, 32, 5, 16, 64, 10),
-                 fwd_frac_bits=None, compare=0, weight_decay_shift=0, rnn_steps=0):
+                 fwd_frac_bits=None, compare=0, weight_decay_shift=0, rnn_steps=0, deal_role=0):
         d = ModelDesc()
         d.kind = kind
         dims = list(dims or ([784, 1] if kind in (LINREG, LOGREG, SVM) else [784, 128, 128, 10]))
@@ -547,6 +555,7 @@ class Model:
         d.compare = compare                           # 0 A2B chain (R9), 1 FSS comparison (R22)
         d.weight_decay_shift = weight_decay_shift     # SVM weight decay (R24)
         d.rnn_steps = rnn_steps                       # RNN sequence length (R25)
+        d.deal_role = deal_role                       # 0 dealer, 1/2 party 0/1 dealing for itself (R23)
         self.ctx, self.desc, self.kind = ctx, d, kind
         h = vp()
         _call("psml_model_create", ctx.handle, ctypes.byref(d), ctypes.byref(h))
@@ -568,6 +577,19 @@ class Model:
 
     def deal(self, step, infer_only=False, stream=None):
         _call("psml_model_deal", self.handle, step, 1 if infer_only else 0, _stream(stream))
+
+    def deal_bundle(self, step, party, stream=None):
+        """Dealer side (deal_role 0): deal `step` and return party `party`'s derived words (R23)."""
+        w = i64()
+        _call("psml_model_deal_bundle", self.handle, step, party, None, ctypes.byref(w), _stream(stream))
+        b = torch.empty(max(w.value, 1), dtype=dtype_of(self.ctx.l), device="cuda")
+        _call("psml_model_deal_bundle", self.handle, step, party, _ptr(b), ctypes.byref(w), _stream(stream))
+        return b[:w.value]
+
+    def deal_party(self, step, party, bundle=None, stream=None):
+        """Party side (deal_role party + 1): own streams + the dealer's bundle (R23)."""
+        n = 0 if bundle is None else bundle.numel()
+        _call("psml_model_deal_party", self.handle, step, party, _ptr(bundle) if n else None, n, _stream(stream))
 
     def train_step(self, X, Y, step, stream=None):
         _call("psml_secure_train_step", self.handle, _pair(X), _pair(Y), step, _stream(stream))

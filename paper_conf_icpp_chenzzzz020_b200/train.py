@@ -40,7 +40,8 @@ class SecureTrainer:
     """One co-resident party pair on the current GPU, training `task` with batch `batch`."""
 
     def __init__(self, task, W_init, batch=128, pair_id=0, dims=None, backend=0,
-                 frac_bits=13, master_frac_bits=27, lr_shift=14, compare="a2b"):
+                 frac_bits=13, master_frac_bits=27, lr_shift=14, compare="a2b", dealer_seed=DEALER_SEED,
+                 deal_role=0, w_shares=None):
         self.task = task
         self.ctx = psml.Ctx(l=64, frac_bits=frac_bits, backend=backend)
         self.ring = self.ctx.ring
@@ -50,10 +51,13 @@ class SecureTrainer:
         rnn = RNN_SHAPE if task == "rnn" else {}
         self.model = psml.Model(self.ctx, KINDS[task], dims=dims or rnn.get("dims"), batch=batch, lr_shift=lr_shift,
                                 rnn_steps=rnn.get("rnn_steps", 0),
-                                master_frac_bits=master_frac_bits, dealer_seed=DEALER_SEED,
+                                master_frac_bits=master_frac_bits, dealer_seed=dealer_seed, deal_role=deal_role,
                                 pair_id=pair_id, fwd_frac_bits=FWD_BITS.get(task),
                                 compare={"a2b": 0, "fss": 1}[compare], weight_decay_shift=WD_SHIFT.get(task, 0))
         for layer, W in enumerate(W_init):
+            if w_shares is not None:   # shares handed over by the client: w_shares[layer] = (Wm_0, Wm_1)
+                self.model.set_master(layer, w_shares[layer])
+                continue
             w = psml.encode(self.master_ring, torch.as_tensor(W, dtype=torch.float64))
             Wm = psml.share(self.ring, SHARE_SEED, call_id(0, INIT_STEP, layer, OP_SHARE, 2), w)
             self.model.set_master(layer, Wm)
@@ -192,11 +196,21 @@ class PartyTrainer(SecureTrainer):
     The dealer runs in each party's process and each party reads only its own half of the
     material (the offline phase a deployment ships from the client)."""
 
-    def __init__(self, task, W_init, party, transport, batch=128, pair_id=0, dp=None, **kw):
+    def __init__(self, task, W_init, party, transport, batch=128, pair_id=0, dp=None, w_share=None, **kw):
+        """w_share: this party's master-weight shares (one tensor per layer) from the client; the
+        model then never holds the peer's share (the peer slot is zero).  Without it the
+        simulation shares W_init itself and then zeroes the peer's slot."""
+        if w_share is not None:
+            kw["w_shares"] = [(w, torch.zeros_like(w)) if party == 0 else (torch.zeros_like(w), w) for w in w_share]
         super().__init__(task, W_init, batch=batch, pair_id=pair_id, **kw)
         self.party = party
         self.xport = transport
         self.dp = dp
+        if w_share is None:   # keep only this party's weight share
+            for layer in range(self.model.n_layers):
+                pair = list(self.model.get_master(layer))
+                pair[1 - party].zero_()
+                self.model.set_master(layer, tuple(pair))
 
     def share_batch(self, X, Y, step):
         """Client role: encode + share; this party receives only its own share."""

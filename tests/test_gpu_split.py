@@ -263,3 +263,78 @@ def test_split_step_cuda_graph_matches_oracle(tmp_path):
     for steps 1..n-1 of two party processes: bit-exact vs the oracle after every step."""
     mp.spawn(_party_graph, args=(_free_port(), str(tmp_path)), nprocs=2, join=True)
     _check_against_oracle(tmp_path, GRAPH_TASKS)
+
+
+# ---------------------------------------------------------------------------------------------
+# Dealer key separation + compressed distribution (DESIGN.md R23): a dealer/client process (this
+# test) holds the dealer seed, deals every step and writes each party's bundle of derived words
+# and its input / weight shares; the two party processes get only their own seed s_i, regenerate
+# their own material, scatter the bundle and train -- bit-exact vs the oracle (which uses the
+# dealer seed), without either party ever holding the dealer seed or the peer's shares.
+# ---------------------------------------------------------------------------------------------
+BUNDLE_TASK, BUNDLE_STEPS = "mlp", 2
+
+
+def _party_bundled(rank, port, outdir, seed_p):
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import synth
+    from paper_conf_icpp_chenzzzz020_b200.parallel import make_dp, make_transport
+    from paper_conf_icpp_chenzzzz020_b200.train import PartyTrainer
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=2)
+    torch.cuda.set_device(0)
+    xp = make_transport(rank, 1 - rank, kind="peer")
+    dp = make_dp([rank], rank)
+    dev = lambda name: torch.from_numpy(np.load(os.path.join(outdir, name))).cuda()  # noqa: E731
+    Wi = synth.init_weights(BUNDLE_TASK)
+    w_share = [dev(f"w{layer}_{rank}.npy") for layer in range(len(Wi))]
+    tr = PartyTrainer(BUNDLE_TASK, Wi, rank, xp, dp=dp, w_share=w_share, dealer_seed=seed_p, deal_role=rank + 1)
+    for s in range(BUNDLE_STEPS):
+        bpath = os.path.join(outdir, f"bundle{s}_{rank}.npy")
+        tr.model.deal_party(s, rank, dev(f"bundle{s}_{rank}.npy") if np.load(bpath).size else None)
+        tr.model.party_train_step(rank, xp, dp, dev(f"x{s}_{rank}.npy"), dev(f"y{s}_{rank}.npy"), s)
+        torch.cuda.synchronize()
+        for layer in range(tr.model.n_layers):
+            np.save(os.path.join(outdir, f"{BUNDLE_TASK}_s{s}_l{layer}_{rank}.npy"), tr.my_master_share(layer).cpu().numpy())
+    tr.close()
+    xp.close()
+    dp.close()
+    dist.destroy_process_group()
+
+
+def test_split_training_with_dealer_bundles(tmp_path):
+    import synth
+    from paper_conf_icpp_chenzzzz020_b200 import build, psml
+    from paper_conf_icpp_chenzzzz020_b200.train import DEALER_SEED, SecureTrainer
+    build.build()
+    torch.cuda.set_device(0)
+    Wi = synth.init_weights(BUNDLE_TASK)
+    dealer = SecureTrainer(BUNDLE_TASK, Wi)          # the client + dealer: holds the dealer seed
+    for layer in range(dealer.model.n_layers):
+        W = dealer.model.get_master(layer)
+        for p in range(2):
+            np.save(tmp_path / f"w{layer}_{p}.npy", W[p].cpu().numpy())
+    sizes = []
+    for s in range(BUNDLE_STEPS):
+        X, Y = synth.batch(BUNDLE_TASK, s)
+        Xs, Ys = dealer.share_batch(torch.from_numpy(X), torch.from_numpy(Y), s)
+        for p in range(2):
+            np.save(tmp_path / f"x{s}_{p}.npy", Xs[p].cpu().numpy())
+            np.save(tmp_path / f"y{s}_{p}.npy", Ys[p].cpu().numpy())
+            b = dealer.model.deal_bundle(s, p)
+            sizes.append(b.numel())
+            np.save(tmp_path / f"bundle{s}_{p}.npy", b.cpu().numpy())
+    torch.cuda.synchronize()
+    dealer.close()
+    assert sizes[0] == 0 and sizes[1] > 0     # party 0 derives all of its A2B-mode material itself
+    seeds = [psml.dealer_party_seed(DEALER_SEED, p) for p in range(2)]
+    port = _free_port()
+    ctx = mp.get_context("spawn")
+    procs = [ctx.Process(target=_party_bundled, args=(p, port, str(tmp_path), seeds[p])) for p in range(2)]
+    for pr in procs:
+        pr.start()
+    for pr in procs:
+        pr.join(600)
+        assert pr.exitcode == 0
+    _check_against_oracle(tmp_path, [(BUNDLE_TASK, BUNDLE_STEPS)])

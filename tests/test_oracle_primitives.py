@@ -106,8 +106,14 @@ def test_triplet_validity(orc, l):
     U = bf.add_mod(U0, U1, l)
     V = bf.add_mod(V0, V1, l)
     assert bf.add_mod(Z0, Z1, l) == bf.matmul_mod(U, V, l)
-    # party 0's bundle is seed-derivable (R4): U0 is exactly the "U0" stream
-    assert np.array_equal(U0.reshape(-1), orc.prg(l, SEED + 2, orc.tag("U0"), 99, M * K))
+    # each party's own streams come from its own seed s_i = PRG(dealer seed, "KD", i) (R4, R23):
+    # U0 / V0 / Z0 from s_0, U1 / V1 from s_1; only Z1 needs both
+    s0, s1 = orc.party_seed(SEED + 2, 0), orc.party_seed(SEED + 2, 1)
+    assert s0 != s1 and SEED + 2 not in (s0, s1)
+    assert s0 == int(orc.prg(64, SEED + 2, orc.tag("KD"), 0, 1)[0])
+    assert np.array_equal(U0.reshape(-1), orc.prg(l, s0, orc.tag("U0"), 99, M * K))
+    assert np.array_equal(Z0.reshape(-1), orc.prg(l, s0, orc.tag("Z0"), 99, M * N))
+    assert np.array_equal(V1.reshape(-1), orc.prg(l, s1, orc.tag("V1"), 99, K * N))
     h = orc.hadamard_triplet_gen(SEED + 2, 100, 50, l)
     for t in range(50):
         u = int(h[0][t]) + int(h[1][t])
@@ -250,3 +256,22 @@ def test_csr_delta_codec(orc):
     assert np.array_equal(orc.delta_csr_apply(prev, enc), cur)
     enc = orc.delta_csr_encode(prev, prev)            # persistent mask, constant data: empty CSR
     assert enc["is_csr"] and enc["nnz"] == 0 and np.array_equal(orc.delta_csr_apply(prev, enc), prev)
+
+
+def test_dealer_key_separation(orc):
+    """DESIGN.md R23: every material stream of party i is keyed by s_i alone; the dealer-only FSS
+    mask stream and the derived words are not reproducible from either party seed."""
+    seed = 0x1234
+    s0, s1 = orc.party_seed(seed, 0), orc.party_seed(seed, 1)
+    for t, want in (("U0", s0), ("V0", s0), ("Z0", s0), ("RA", s0), ("FS", s0), ("F0", s0), ("K0", s0),
+                    ("U1", s1), ("V1", s1), ("R1", s1), ("K1", s1), ("FR", seed)):
+        assert orc.stream_seed(seed, orc.tag(t)) == want, t
+    for t in range(12):   # boolean AND triplet streams a_i^t, b_i^t, c_0^t
+        assert orc.stream_seed(seed, orc.tag(bytes([ord("a"), ord("0"), t]))) == s0
+        assert orc.stream_seed(seed, orc.tag(bytes([ord("b"), ord("1"), t]))) == s1
+        assert orc.stream_seed(seed, orc.tag(bytes([ord("c"), ord("0"), t]))) == s0
+    m0, m1 = orc.msb_dealer(seed, 5, 64)
+    n = 64
+    # party 1's a/b words from s_1 alone; its c words are derived (need a_0, b_0 too)
+    assert np.array_equal(m1[:n], orc.prg(64, s1, orc.tag(bytes([ord("a"), ord("1"), 0])), 5, n))
+    assert not np.array_equal(m1[2 * n:3 * n], orc.prg(64, s1, orc.tag(bytes([ord("c"), ord("1"), 0])), 5, n))
