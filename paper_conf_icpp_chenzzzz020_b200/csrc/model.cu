@@ -1677,7 +1677,7 @@ psml_status psml_model_deal_party(psml_model m, uint32_t step_id, int32_t party,
     for (auto &r : derived_regions(m, pool, party)) tot += r.second;
     if (words != tot) return fail(PSML_ERR_SHAPE, "bundle size does not match this model's derived words");
     if (tot && !bundle) return fail(PSML_ERR_INVALID, "bundle is null");
-    PSML_TRY(check_ptrs({bundle}));
+    if (tot) PSML_TRY(check_ptrs({bundle}));
     PSML_TRY(psml_model_deal(m, step_id, 0, stream));   // this party's own streams (the rest is junk)
     const T *in = (const T *)bundle;
     for (auto &r : derived_regions(m, pool, party)) {

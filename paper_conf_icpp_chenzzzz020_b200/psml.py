@@ -183,9 +183,22 @@ def _ptr(t):
 
 
 def _pair(ts):
+    """A pair of device pointers; every tensor must be a contiguous CUDA tensor (no CPU fallback,
+    and the C ABI takes sizes from its own arguments, so a wrong tensor must not reach it)."""
     if ts is None:
         return None
-    return P2(*(None if t is None else t.data_ptr() for t in ts))
+    return P2(*(None if t is None else _ptr(t).value for t in ts))
+
+
+def _check(ts, words, dtypes, what):
+    """Shape / dtype guard for model-sized buffers (the ABI reads `words` elements from each)."""
+    for t in ([ts] if torch.is_tensor(ts) else list(ts)):
+        if t is None:
+            continue
+        if t.dtype not in dtypes:
+            raise PsmlError("marshal", 1, f"{what}: dtype {t.dtype}, expected one of {dtypes}")
+        if t.numel() != words:
+            raise PsmlError("marshal", 2, f"{what}: {t.numel()} elements, expected {words}")
 
 
 def _stream(stream=None):
@@ -561,6 +574,12 @@ class Model:
         _call("psml_model_create", ctx.handle, ctypes.byref(d), ctypes.byref(h))
         self.handle = h
         self.n_layers = d.n_layers
+        # words per minibatch of one party's input / label shares (guards the ABI calls)
+        x_row = (cnn[0] * cnn[1] * cnn[2] if kind == CNN else
+                 (rnn_steps * dims[0] if kind == RNN else dims[0]))
+        self.x_words = batch * x_row
+        self.y_words = batch * self.layer_shape(self.n_layers - 1)[1]
+        self.ring_dtypes = (dtype_of(ctx.l), torch.int64 if ctx.l == 64 else torch.int32)
 
     def layer_shape(self, layer):
         r, c = i64(), i64()
@@ -591,10 +610,16 @@ class Model:
         n = 0 if bundle is None else bundle.numel()
         _call("psml_model_deal_party", self.handle, step, party, _ptr(bundle) if n else None, n, _stream(stream))
 
+    def _xy(self, X, Y):
+        _check(X, self.x_words, self.ring_dtypes, "X shares")
+        _check(Y, self.y_words, self.ring_dtypes, "Y shares")
+
     def train_step(self, X, Y, step, stream=None):
+        self._xy(X, Y)
         _call("psml_secure_train_step", self.handle, _pair(X), _pair(Y), step, _stream(stream))
 
     def forward_backward(self, X, Y, step, stream=None):
+        self._xy(X, Y)
         _call("psml_train_forward_backward", self.handle, _pair(X), _pair(Y), step,
               _stream(stream))
 
@@ -619,6 +644,7 @@ class Model:
         the dealer of step s + 1 overlaps the online phase of step s).  unsafe_reuse_material
         (benchmark-only timing of the online phase): replay the material dealt once into pool 0
         on every step -- never in a real run, reused masks leak."""
+        self._xy(X, Y)
         flags = ((1 if with_deal else 0) | (2 if with_update else 0) | (4 if pipelined else 0)
                  | (8 if unsafe_reuse_material else 0))
         _call("psml_model_capture_step", self.handle, _pair(X), _pair(Y), flags, _stream(stream))
@@ -636,23 +662,31 @@ class Model:
         a (2, batch, d_L) uint64 CPU tensor -- all host tensors (pinned)."""
         if q.dtype != torch.uint8 or y.dtype not in (torch.uint8, torch.float64) or yhat_host.dtype != torch.uint64:
             raise PsmlError("marshal", 1, "step_host: q uint8, y float64 | uint8, yhat_host uint64")
+        batch = self.desc.batch
+        want_y = batch if y.dtype == torch.uint8 else self.y_words
+        if q.numel() != self.x_words or y.numel() != want_y or yhat_host.numel() < 2 * self.y_words:
+            raise PsmlError("marshal", 2, f"step_host: q {q.numel()} (want {self.x_words}), y {y.numel()} "
+                                          f"(want {want_y}), yhat_host {yhat_host.numel()} (want >= {2 * self.y_words})")
         _call("psml_model_step_host", self.handle, _host_ptr(q), _host_ptr(y), 1 if y.dtype == torch.uint8 else 0,
               share_seed, step, _host_ptr(yhat_host), _stream(stream))
 
     def party_train_step(self, party, xport, dp, X_i, Y_i, step, stream=None):
         """Split deployment: forward/backward + this party's gradient all-reduce over `dp`
         (DataParallel or None) + update (psml_party_train_step)."""
+        self._xy(X_i, Y_i)
         _call("psml_party_train_step", self.handle, party, xport.handle, dp.handle if dp else None,
               _ptr(X_i), _ptr(Y_i), step, _stream(stream))
 
     def party_capture_step(self, party, xport, dp, X_i, Y_i, with_deal=True, with_update=True,
                            pipelined=False, stream=None):
+        self._xy(X_i, Y_i)
         flags = (1 if with_deal else 0) | (2 if with_update else 0) | (4 if pipelined else 0)
         _call("psml_party_capture_step", self.handle, party, xport.handle, dp.handle if dp else None,
               _ptr(X_i), _ptr(Y_i), flags, _stream(stream))
 
     def party_forward_backward(self, party, xport, X_i, Y_i, step, stream=None):
         """Split deployment: party `party`'s half of the step, openings through `xport`."""
+        self._xy(X_i, Y_i)
         _call("psml_party_forward_backward", self.handle, party, xport.handle, _ptr(X_i), _ptr(Y_i),
               step, _stream(stream))
 
@@ -660,7 +694,9 @@ class Model:
         _call("psml_party_apply_update", self.handle, party, extra_shift, _stream(stream))
 
     def infer(self, X, step, out_shape, stream=None):
+        _check(X, self.x_words, self.ring_dtypes, "X shares")
         Y = empty_pair(out_shape, self.ctx.l)
+        _check(Y, self.y_words, self.ring_dtypes, "prediction buffers")
         _call("psml_secure_infer", self.handle, _pair(X), step, _pair(Y), _stream(stream))
         return Y
 

@@ -35,3 +35,18 @@ def test_no_gpu_fails_loudly():
     assert e.value.status == 4  # PSML_ERR_UNSUPPORTED, never a CPU fallback
     assert psml.msb_material_words(psml.Ring(64, 13), 10) == (6 * 6 + 2) * 10
     assert psml.msb_material_words(psml.Ring(32, 13), 10) == (6 * 5 + 2) * 10
+
+
+def test_binding_rejects_wrong_buffers_before_the_abi():
+    """the binding checks device, contiguity, dtype and element count before a
+    pointer reaches the C ABI (which takes sizes from the model description)."""
+    import torch
+    from paper_conf_icpp_chenzzzz020_b200 import psml
+    cpu = torch.zeros(4, dtype=torch.uint64)
+    with pytest.raises(psml.PsmlError):
+        psml._pair((cpu, cpu))
+    with pytest.raises(psml.PsmlError):
+        psml._check(torch.zeros(10, dtype=torch.uint64), 12, (torch.uint64,), "X")
+    with pytest.raises(psml.PsmlError):
+        psml._check(torch.zeros(12, dtype=torch.float64), 12, (torch.uint64,), "X")
+    psml._check(torch.zeros(12, dtype=torch.uint64), 12, (torch.uint64,), "X")
