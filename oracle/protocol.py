@@ -108,8 +108,10 @@ def sub_pair(a, b):
 class Model:
     """Both parties' weight shares: master (MASTER fractional bits) and forward copy (fw[l] bits)."""
 
-    def __init__(self, task, W_init, fw=None, compare="a2b"):
+    def __init__(self, task, W_init, fw=None, compare="a2b", mask_reuse=False):
         self.task = task
+        self.mask_reuse = mask_reuse   # SecureML forward/backward mask reuse (R26; MLP family only)
+        assert not mask_reuse or task in ("linreg", "logreg", "mlp")
         self.compare = compare   # secure comparison of ReLU / Eq. 9: "a2b" (R9) or "fss" (R22)
         self.fw = list(fw) if fw is not None else list(FWD_BITS[task])
         if task == "mlp" and fw is None:
@@ -130,6 +132,32 @@ class Model:
 # ---------------------------------------------------------------------------------------------
 def _T(p):
     return np.ascontiguousarray(p[0].T), np.ascontiguousarray(p[1].T)
+
+
+def reuse_triplets(pair, step, layer, B, din, dout):
+    """SecureML forward/backward mask reuse (R26): the backward
+    products of layer l re-use the masks of values already opened -- the activation A_l's forward
+    mask U_f (gradW's left operand A_l^T - U_f^T = E_f^T) and the weight's forward mask V_f (gradin's
+    right operand W_l^T - V_f^T = F_f^T) -- and ONE fresh mask D of delta serves both products
+    (gradW's right operand and gradin's left operand).  D_i = PRG("U0"/"U1") and Z_0 = PRG("Z0")
+    under the gradin call id, Z_0 of gradW under the gradW call id; Z_1 = U V - Z_0 as usual.
+    Returns (gradW triplet, gradin triplet) in core.triplet_gen's (U0, U1, V0, V1, Z0, Z1) order."""
+    Uf0, Uf1, Vf0, Vf1, _, _ = core.triplet_gen(DEALER_SEED, call_id(pair, step, layer, OP_FWD, 0), B, din, dout, L)
+    cgi, cgw = call_id(pair, step, layer, OP_GRADIN, 0), call_id(pair, step, layer, OP_GRADW, 0)
+    D0 = core.dealer_prg(L, DEALER_SEED, core.tag("U0"), cgi, B * dout).reshape(B, dout)
+    D1 = core.dealer_prg(L, DEALER_SEED, core.tag("U1"), cgi, B * dout).reshape(B, dout)
+    Ug = (np.ascontiguousarray(Uf0.T), np.ascontiguousarray(Uf1.T))
+    Zg = core.ring_matmul(np.ascontiguousarray((Uf0 + Uf1).T), D0 + D1)
+    Zg0 = core.dealer_prg(L, DEALER_SEED, core.tag("Z0"), cgw, din * dout).reshape(din, dout)
+    Vi = (np.ascontiguousarray(Vf0.T), np.ascontiguousarray(Vf1.T))
+    Zi = core.ring_matmul(D0 + D1, np.ascontiguousarray((Vf0 + Vf1).T))
+    Zi0 = core.dealer_prg(L, DEALER_SEED, core.tag("Z0"), cgi, B * din).reshape(B, din)
+    return ((Ug[0], Ug[1], D0, D1, Zg0, Zg - Zg0), (D0, D1, Vi[0], Vi[1], Zi0, Zi - Zi0))
+
+
+def matmul_with(A, B, trip, trunc):
+    c = core.beaver_matmul(A, B, trip, trunc=0, l=L)
+    return checked_trunc(c, trunc) if trunc else c
 
 
 def matmul(A, B, pair, step, layer, op, trunc):
@@ -327,7 +355,16 @@ def forward_backward(model, Xs, Ys, step, pair=0):
     yhat = h
     delta = sub_pair(yhat, Ys)
     grads = [None] * nl
+    B = Xs[0].shape[0]
     for layer in range(nl - 1, -1, -1):
+        if model.mask_reuse:
+            din, dout = model.W[layer][0].shape
+            tg, ti = reuse_triplets(pair, step, layer, B, din, dout)
+            grads[layer] = matmul_with(_T(acts[layer]), delta, tg, 0)
+            if layer > 0:
+                t = matmul_with(delta, _T(model.W[layer]), ti, model.fw[layer])
+                delta = hadamard(t, drelus[layer - 1], pair, step, layer - 1, 1)
+            continue
         grads[layer] = matmul(_T(acts[layer]), delta, pair, step, layer, OP_GRADW, 0)
         if layer > 0:
             t = matmul(delta, _T(model.W[layer]), pair, step, layer, OP_GRADIN, model.fw[layer])

@@ -359,3 +359,34 @@ def test_rnn_training_tracks_fp64_and_inference():
     for t in range(16):
         h = np.maximum(np.concatenate([Xq[:, 32 * t:32 * (t + 1)], h], axis=1) @ W1, 0.0)
     assert np.abs(got - plain.eq9(h @ Wo)).max() < 2.0 ** -8
+
+
+def test_mask_reuse_triplets_and_openings(orc):
+    """R26: the reuse triplets are valid triplets (Z_0 + Z_1 = U V), and the backward products'
+    re-used operands open to exactly the forward openings transposed: E_gradW = E_fwd^T,
+    F_gradin = F_fwd^T, and delta is opened once (F_gradW = E_gradin)."""
+    B, din, dout, layer, step = 8, 12, 5, 1, 3
+    A = orc.share(orc.prg(64, 1, orc.tag("ra"), 0, B * din).reshape(B, din), 2, 0)
+    W = orc.share(orc.prg(64, 1, orc.tag("rw"), 0, din * dout).reshape(din, dout), 2, 1)
+    D = orc.share(orc.prg(64, 1, orc.tag("rd"), 0, B * dout).reshape(B, dout), 2, 2)
+    tg, ti = P.reuse_triplets(0, step, layer, B, din, dout)
+    for t in (tg, ti):
+        assert np.array_equal(t[4] + t[5], orc.ring_matmul(t[0] + t[1], t[2] + t[3]))
+    tf = orc.triplet_gen(P.DEALER_SEED, P.call_id(0, step, layer, P.OP_FWD, 0), B, din, dout)
+    _, trf = orc.beaver_matmul(A, W, tf, trace=True)
+    _, trg = orc.beaver_matmul(P._T(A), D, tg, trace=True)
+    _, tri = orc.beaver_matmul(D, P._T(W), ti, trace=True)
+    assert np.array_equal(trg["E"], trf["E"].T) and np.array_equal(tri["F"], trf["F"].T)
+    assert np.array_equal(trg["F"], tri["E"])
+
+
+@pytest.mark.parametrize("task,steps", [("logreg", 20), ("mlp", 4)])
+def test_mask_reuse_training_tracks_fp64(task, steps):
+    Wi = synth.init_weights(task)
+    m, pm = P.Model(task, Wi, mask_reuse=True), plain.PlainModel(task, Wi)
+    for s in range(steps):
+        X, Y = synth.batch(task, s)
+        P.train_step(m, X, Y, s)
+        pm.step(X, Y)
+    err = max(np.abs(a - b).max() for a, b in zip(m.decoded_master(), pm.W))
+    assert err < 2.0 ** -15, np.log2(err)
