@@ -306,6 +306,10 @@ typedef struct {
     int32_t weight_decay_shift; /* 0 = none; else W^m -= trunc(W^m, shift) every update (SVM:
                                    lambda.eta = 2^-16, R24)                        */
     int32_t rnn_steps;        /* RNN: sequence length T (1..254; call-id layers 1..T+1)       */
+    int32_t mask_reuse;       /* DESIGN.md R26 (linear / logistic regression, MLP): the backward
+                                 products re-use the forward masks of A_l and W_l and one fresh
+                                 mask of delta, so the split engine opens delta once per layer
+                                 instead of re-opening A^T, W^T and delta twice                */
     int32_t deal_role;        /* DESIGN.md R23: 0 = the dealer (dealer_seed = the dealer seed; every
                                  stream), 1 / 2 = party 0 / 1 dealing for itself (dealer_seed =
                                  that party's seed s_i = psml_dealer_party_seed(dealer seed, i));

@@ -160,6 +160,10 @@ struct psml_model_s {
     // RNN (R25): per time step inputs A_t = [x_t | h_{t-1}], states h_t, DReLU_t, and the
     // per-step weight-gradient product before it is added into the layer-0 gradient
     psml::Buf rnnA, rnnH, rnnD, rnnG;
+    // split engine with mask reuse (R26): this party's copy of each layer's forward openings E, F,
+    // the opened delta, and scratch (transposes, a zero operand, delta's send / receive messages)
+    std::vector<psml::T *> eopen, fopen;
+    psml::T *dopen = nullptr, *rT = nullptr, *rzero = nullptr, *dms = nullptr, *dmr = nullptr;
     int rnn_T = 0, rnn_D = 0;
     psml_xport cap_xport = nullptr;
     psml_dp cap_dp = nullptr;
@@ -399,9 +403,52 @@ static psml_status deal_gemm(psml_model_s *m, DealItem &it, cudaStream_t s) {
     return launch_ring_gemm<T, ConvDealerOps<T>>(ops, m->dws, m->dws_words, s, m->ctx->sm_count);
 }
 
+// out_p = transpose(in_p): in is R x C row-major, out C x R (both parties)
+static __global__ void transpose_pair_kernel(CPair<T> in, int64_t R, int64_t C, Pair<T> out) {
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < R * C; e += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r = e / C, c = e % C;
+#pragma unroll
+        for (int p = 0; p < 2; ++p) out.p[p][c * R + r] = in.p[p][e];
+    }
+}
+
+// SecureML mask reuse (R26): the backward triplets of layer l copy the forward masks --
+// gradW: U = U_f^T, V = D;  gradin: U = D, V = V_f^T -- with D = PRG("U0"/"U1") under the gradin
+// call id; Z_0 = PRG("Z0") under the item's own call id and Z_1 = U V - Z_0 as usual.
+static psml_status deal_reuse_item(psml_model_s *m, DealItem &it, uint32_t step, cudaStream_t s) {
+    DealItem *f = nullptr;   // the forward triplet of the same layer in the same pool as `it`
+    for (auto &items : m->items)
+        if (&it >= items.data() && &it < items.data() + items.size())
+            for (auto &x : items)
+                if (x.layer == it.layer && x.op == OP_FWD && x.kind == IT_MATRIX) f = &x;
+    if (!f) return fail(PSML_ERR_STATE, "mask reuse: missing forward triplet");
+    const DealSeeds &S = m->seeds;
+    const uint64_t cgi = call_id(m->d.pair_id, step, it.layer, OP_GRADIN, 0);
+    const uint64_t cid = call_id(m->d.pair_id, step, it.layer, it.op, it.slot);
+    const int64_t B = f->M, din = f->K, dout = f->N;
+    Buf &D = it.op == OP_GRADW ? it.V : it.U;   // B x dout
+    dealer_pair_kernel<T><<<grid_for(D.n / 8 + 1, 256), 256, 0, s>>>(dkey(S, TAG_U0, cgi, m->step_dev),
+                                                                     dkey(S, TAG_U1, cgi, m->step_dev), D.n, D.p[0],
+                                                                     D.p[1], nullptr);
+    PSML_LAUNCH_CHECK();
+    if (it.op == OP_GRADW)   // U = U_f^T (din x B)
+        transpose_pair_kernel<<<ew_grid(B * din), EW_THREADS, 0, s>>>(CPair<T>{{f->U.p[0], f->U.p[1]}}, B, din,
+                                                                      Pair<T>{{it.U.p[0], it.U.p[1]}});
+    else                     // V = V_f^T (dout x din)
+        transpose_pair_kernel<<<ew_grid(din * dout), EW_THREADS, 0, s>>>(CPair<T>{{f->V.p[0], f->V.p[1]}}, din, dout,
+                                                                         Pair<T>{{it.V.p[0], it.V.p[1]}});
+    PSML_LAUNCH_CHECK();
+    prg_kernel<T, 0><<<grid_for(it.Z.n / 8 + 2, 256), 256, 0, s>>>(dkey(S, TAG_Z0, cid, m->step_dev), 0, it.Z.n,
+                                                                     it.Z.p[0], nullptr, nullptr);
+    PSML_LAUNCH_CHECK();
+    return deal_gemm(m, it, s);
+}
+
 static psml_status deal_item(psml_model_s *m, DealItem &it, uint32_t step, cudaStream_t s) {
     const uint64_t seed = m->d.dealer_seed;
     const uint64_t cid = call_id(m->d.pair_id, step, it.layer, it.op, it.slot);
+    if (m->d.mask_reuse && it.kind == IT_MATRIX && (it.op == OP_GRADW || it.op == OP_GRADIN))
+        return deal_reuse_item(m, it, step, s);
     switch (it.kind) {
     case IT_MATRIX:
     case IT_CONV_FWD:
@@ -561,7 +608,7 @@ static psml_status deal_prg_launch(psml_model_s *m, const DealPlan &P, int j0, i
 // material is ready early; s joins s2 before returning.
 static psml_status deal_pool(psml_model_s *m, int pool, uint32_t step, bool infer_only, cudaStream_t s,
                              cudaStream_t s2 = nullptr) {
-    if (!fused_deal()) {
+    if (!fused_deal() || m->d.mask_reuse) {   // mask reuse: the backward triplets copy forward masks
         for (auto &it : m->items[pool]) {
             if (infer_only && !it.fwd) continue;
             PSML_TRY(deal_item(m, it, step, s));
@@ -889,6 +936,7 @@ static bool fused_eligible(const psml_model_s *m) {
     for (int l = 0; l < m->nl; ++l)
         if (fw(m, l) != m->ctx->ring.frac_bits) return false;   // the fused step truncates by F
     if (m->d.compare != 0) return false;                         // the fused step runs the A2B chain
+    if (m->d.mask_reuse) return false;                           // ... and fresh backward masks
     return fuse_enabled() && chain_mode() == 0;
 }
 
@@ -1115,6 +1163,19 @@ static psml_status forward_backward(psml_model_s *m, const T *const X[2], const 
 // opens send + recv.  The round kernels are the co-resident ones restricted to party `only`
 // (kernels.cuh), so shares and opened values are bit-identical to the co-resident engine.
 // ------------------------------------------------------------------------------------------------
+static __global__ void add_one_kernel(const T *a, const T *b, int64_t n, T *c) {
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x)
+        c[e] = a[e] + b[e];
+}
+static __global__ void sub_one_kernel(const T *a, const T *b, int64_t n, T *c) {
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x)
+        c[e] = a[e] - b[e];
+}
+static __global__ void transpose_one_kernel(const T *in, int64_t R, int64_t C, T *out) {
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < R * C; e += (int64_t)gridDim.x * blockDim.x)
+        out[(e % C) * R + e / C] = in[e];
+}
+
 struct PartyRun {
     psml_model_s *m;
     int p;            // this party
@@ -1163,8 +1224,42 @@ static psml_status party_mm(PartyRun &r, const T *A, const T *Bm, int layer, int
     const psml_stream ps = (psml_stream)r.s;
     PSML_TRY(psml_beaver_mask(ctx, r.p, A, Bm, it->U.p[r.p], it->V.p[r.p], M, K, N, flags, Es, Fs, ps));
     PSML_TRY(xchg(r, {{Es, Er, M * K}, {Fs, Fr, K * N}}));
+    if (m->d.mask_reuse && op == OP_FWD) {   // keep this layer's openings for the backward products (R26)
+        add_one_kernel<<<ew_grid(M * K), EW_THREADS, 0, r.s>>>(Es, Er, M * K, m->eopen[layer]);
+        PSML_LAUNCH_CHECK();
+        add_one_kernel<<<ew_grid(K * N), EW_THREADS, 0, r.s>>>(Fs, Fr, K * N, m->fopen[layer]);
+        PSML_LAUNCH_CHECK();
+    }
     return psml_beaver_open_matmul(ctx, r.p, Es, Er, Fs, Fr, it->U.p[r.p], it->V.p[r.p], it->Z.p[r.p], M, K, N, trunc,
                                    C, ps);
+}
+
+// Backward products of layer l with mask reuse (R26): ONE exchange (delta_i - D_i); gradW opens to
+// (E_f^T, delta) and gradin to (delta, F_f^T) from this party's stored forward openings.
+static psml_status party_backward_reuse(PartyRun &r, int l, const T *delta, T *gW, T *gin, int trunc) {
+    psml_model_s *m = r.m;
+    const int p = r.p;
+    DealItem *g = find_item(m, l, OP_GRADW, 0), *gi = l > 0 ? find_item(m, l, OP_GRADIN, 0) : nullptr;
+    if (!g || (l > 0 && !gi)) return fail(PSML_ERR_STATE, "missing backward triplet");
+    const int64_t B = m->B, din = m->rows[l], dout = m->cols[l];
+    psml_ctx ctx = reinterpret_cast<psml_ctx>(m->ctx);
+    const psml_stream ps = (psml_stream)r.s;
+    sub_one_kernel<<<ew_grid(B * dout), EW_THREADS, 0, r.s>>>(delta, g->V.p[p], B * dout, m->dms);   // delta_i - D_i
+    PSML_LAUNCH_CHECK();
+    PSML_TRY(xchg(r, {{m->dms, m->dmr, B * dout}}));
+    add_one_kernel<<<ew_grid(B * dout), EW_THREADS, 0, r.s>>>(m->dms, m->dmr, B * dout, m->dopen);
+    PSML_LAUNCH_CHECK();
+    // gradW = A^T . delta: E = E_f^T (din x B), F = delta
+    transpose_one_kernel<<<ew_grid(B * din), EW_THREADS, 0, r.s>>>(m->eopen[l], B, din, m->rT);
+    PSML_LAUNCH_CHECK();
+    PSML_TRY(psml_beaver_open_matmul(ctx, p, m->rT, m->rzero, m->dopen, m->rzero, g->U.p[p], g->V.p[p], g->Z.p[p], din, B,
+                                     dout, 0, gW, ps));
+    if (!gi) return PSML_OK;
+    // gradin = delta . W^T: E = delta, F = F_f^T (dout x din)
+    transpose_one_kernel<<<ew_grid(din * dout), EW_THREADS, 0, r.s>>>(m->fopen[l], din, dout, m->rT);
+    PSML_LAUNCH_CHECK();
+    return psml_beaver_open_matmul(ctx, p, m->dopen, m->rzero, m->rT, m->rzero, gi->U.p[p], gi->V.p[p], gi->Z.p[p], B,
+                                   dout, din, trunc, gin, ps);
 }
 
 // FSS comparison (R22), one party: round 1 exchanges x_i + r_i, the DCF evaluation gives DReLU,
@@ -1383,11 +1478,14 @@ static psml_status party_forward_backward(PartyRun &r, const T *X, const T *Y) {
     T *g[2];
     for (int l = nl - 1; l >= 0; --l) {
         gradp(m, l, g);
-        PSML_TRY(party_mm(r, m->act[l].p[p], m->delta.p[p], l, OP_GRADW, PSML_TRANS_A, 0, g[p]));
-        if (l > 0) {
-            PSML_TRY(party_mm(r, m->delta.p[p], m->W[l].p[p], l, OP_GRADIN, PSML_TRANS_B, fw(m, l), m->tmp.p[p]));
-            PSML_TRY(party_had(r, m->tmp.p[p], m->drelu[l - 1].p[p], l - 1, 1, m->delta.p[p]));
+        if (m->d.mask_reuse) {
+            PSML_TRY(party_backward_reuse(r, l, m->delta.p[p], g[p], m->tmp.p[p], fw(m, l)));
+        } else {
+            PSML_TRY(party_mm(r, m->act[l].p[p], m->delta.p[p], l, OP_GRADW, PSML_TRANS_A, 0, g[p]));
+            if (l > 0)
+                PSML_TRY(party_mm(r, m->delta.p[p], m->W[l].p[p], l, OP_GRADIN, PSML_TRANS_B, fw(m, l), m->tmp.p[p]));
         }
+        if (l > 0) PSML_TRY(party_had(r, m->tmp.p[p], m->drelu[l - 1].p[p], l - 1, 1, m->delta.p[p]));
     }
     return PSML_OK;
 }
@@ -1462,6 +1560,8 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
     default:
         return fail(PSML_ERR_INVALID, "unknown model kind");
     }
+    if (desc->mask_reuse && desc->kind != PSML_LINREG && desc->kind != PSML_LOGREG && desc->kind != PSML_MLP)
+        return fail(PSML_ERR_UNSUPPORTED, "mask_reuse: linear / logistic regression and MLP");
     if (desc->weight_decay_shift < 0 || desc->weight_decay_shift >= 64)
         return fail(PSML_ERR_INVALID, "weight_decay_shift must be in [0, 64)");
     for (int l = 0; l < m->nl; ++l) {
@@ -1497,6 +1597,24 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
     PSML_TRY(balloc(mp, m->yhat, B * m->dims[m->nl]));
     PSML_TRY(balloc(mp, m->delta, B * maxw));
     PSML_TRY(balloc(mp, m->tmp, B * std::max<int64_t>(maxw, 3)));   // SVM: margin, indicator, y (.) ind
+    if (m->d.mask_reuse) {
+        int64_t mx = 0, bo = 0;
+        m->eopen.assign(m->nl, nullptr);
+        m->fopen.assign(m->nl, nullptr);
+        for (int l = 0; l < m->nl; ++l) {
+            PSML_TRY(dalloc(mp, &m->eopen[l], B * m->rows[l]));
+            PSML_TRY(dalloc(mp, &m->fopen[l], m->rows[l] * m->cols[l]));
+            mx = std::max(mx, std::max(B * m->rows[l], m->rows[l] * m->cols[l]));
+            bo = std::max(bo, B * m->cols[l]);
+        }
+        mx = std::max(mx, bo);
+        PSML_TRY(dalloc(mp, &m->dopen, bo));
+        PSML_TRY(dalloc(mp, &m->dms, bo));
+        PSML_TRY(dalloc(mp, &m->dmr, bo));
+        PSML_TRY(dalloc(mp, &m->rT, mx));
+        PSML_TRY(dalloc(mp, &m->rzero, mx));
+        PSML_CUDA_TRY(cudaMemset(m->rzero, 0, sizeof(T) * mx));
+    }
     if (m->d.kind == PSML_RNN) {
         const int64_t T = m->rnn_T, H = m->dims[1];
         PSML_TRY(balloc(mp, m->rnnA, T * B * m->rows[0]));

@@ -41,7 +41,7 @@ class SecureTrainer:
 
     def __init__(self, task, W_init, batch=128, pair_id=0, dims=None, backend=0,
                  frac_bits=13, master_frac_bits=27, lr_shift=14, compare="a2b", dealer_seed=DEALER_SEED,
-                 deal_role=0, w_shares=None):
+                 deal_role=0, w_shares=None, mask_reuse=False):
         self.task = task
         self.ctx = psml.Ctx(l=64, frac_bits=frac_bits, backend=backend)
         self.ring = self.ctx.ring
@@ -53,7 +53,8 @@ class SecureTrainer:
                                 rnn_steps=rnn.get("rnn_steps", 0),
                                 master_frac_bits=master_frac_bits, dealer_seed=dealer_seed, deal_role=deal_role,
                                 pair_id=pair_id, fwd_frac_bits=FWD_BITS.get(task),
-                                compare={"a2b": 0, "fss": 1}[compare], weight_decay_shift=WD_SHIFT.get(task, 0))
+                                compare={"a2b": 0, "fss": 1}[compare], weight_decay_shift=WD_SHIFT.get(task, 0),
+                                mask_reuse=mask_reuse)
         for layer, W in enumerate(W_init):
             if w_shares is not None:   # shares handed over by the client: w_shares[layer] = (Wm_0, Wm_1)
                 self.model.set_master(layer, w_shares[layer])

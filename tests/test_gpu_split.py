@@ -158,9 +158,10 @@ def test_split_compressed_transmission(tmp_path):
 # ---------------------------------------------------------------------------------------------
 SPLIT_TASKS = [("linreg", 2), ("logreg", 2), ("mlp", 2), ("cnn", 1)]
 FSS_TASKS = [("logreg", 2), ("mlp", 2)]
+REUSE_TASKS = [("linreg", 2), ("mlp", 2)]
 
 
-def _party_train(rank, port, outdir, kind, compare="a2b"):
+def _party_train(rank, port, outdir, kind, compare="a2b", mask_reuse=False):
     import sys
     sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
     import synth
@@ -171,8 +172,10 @@ def _party_train(rank, port, outdir, kind, compare="a2b"):
     torch.cuda.set_device(0)
     xp = make_transport(rank, 1 - rank, kind=kind)
     dp = make_dp([rank], rank)          # one pair: the party's data-parallel group is itself
-    for task, steps in (SPLIT_TASKS if compare == "a2b" else FSS_TASKS):
-        tr = PartyTrainer(task, synth.init_weights(task), rank, xp, backend=1, dp=dp, compare=compare)
+    tasks = REUSE_TASKS if mask_reuse else (SPLIT_TASKS if compare == "a2b" else FSS_TASKS)
+    for task, steps in tasks:
+        tr = PartyTrainer(task, synth.init_weights(task), rank, xp, backend=1, dp=dp, compare=compare,
+                          mask_reuse=mask_reuse)
         for s in range(steps):
             X, Y = synth.batch(task, s)
             tr.step(torch.from_numpy(X), torch.from_numpy(Y), s)
@@ -188,11 +191,11 @@ def _party_train(rank, port, outdir, kind, compare="a2b"):
     dist.destroy_process_group()
 
 
-def _check_against_oracle(tmp_path, tasks, compare="a2b"):
+def _check_against_oracle(tmp_path, tasks, compare="a2b", mask_reuse=False):
     import synth
     from oracle import protocol as OP
     for task, steps in tasks:
-        om = OP.Model(task, synth.init_weights(task), compare=compare)
+        om = OP.Model(task, synth.init_weights(task), compare=compare, mask_reuse=mask_reuse)
         for s in range(steps):
             X, Y = synth.batch(task, s)
             OP.train_step(om, X, Y, s)
@@ -221,6 +224,13 @@ def test_split_training_fss_comparison_matches_oracle(tmp_path):
     _check_against_oracle(tmp_path, FSS_TASKS, compare="fss")
     st = [np.load(tmp_path / f"xstats_{p}.npy") for p in range(2)]
     assert st[0][1] == st[1][1] > 0
+
+
+def test_split_training_mask_reuse_matches_oracle(tmp_path):
+    """Mask reuse in the split engine (R26): the backward products open delta once per layer and
+    reuse this party's stored forward openings; fewer exchanges and bytes, bit-exact vs the oracle."""
+    mp.spawn(_party_train, args=(_free_port(), str(tmp_path), "peer", "a2b", True), nprocs=2, join=True)
+    _check_against_oracle(tmp_path, REUSE_TASKS, mask_reuse=True)
 
 
 GRAPH_TASKS = [("mlp", 4), ("logreg", 3)]

@@ -235,3 +235,25 @@ def test_seg_gemm_backends_match_oracle(env):
                         os.path.join(root, "tests", "test_gpu_primitives.py")],
                        env=env, capture_output=True, text=True, cwd=root)
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
+
+
+@pytest.mark.parametrize("task", ["logreg", "mlp"])
+def test_mask_reuse_bitexact_vs_oracle(T, task):
+    """SecureML forward/backward mask reuse (R26): eager step, then pipelined CUDA-graph
+    replays (dealer inside the graph), bit-exact vs the oracle's reuse protocol."""
+    Wi = synth.init_weights(task)
+    tr = T.SecureTrainer(task, Wi, backend=1, mask_reuse=True)
+    om = OP.Model(task, Wi, mask_reuse=True)
+    X, Y = synth.batch(task, 0)
+    tr.step(torch.from_numpy(X), torch.from_numpy(Y), 0)
+    OP.train_step(om, X, Y, 0)
+    torch.cuda.synchronize()
+    _compare_shares(tr, om)
+    tr.capture(pipelined=True)
+    for s in range(1, 3):
+        X, Y = synth.batch(task, s)
+        tr.graph_step(torch.from_numpy(X), torch.from_numpy(Y), s)
+        OP.train_step(om, X, Y, s)
+        torch.cuda.synchronize()
+        _compare_shares(tr, om)
+    tr.close()
