@@ -49,6 +49,10 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-ring-gemm", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--mask-reuse", action="store_true",
+                    help="split deployment: SecureML forward/backward mask reuse (DESIGN.md R26)")
+    ap.add_argument("--compare", default="a2b", choices=["a2b", "fss"],
+                    help="secure comparison of ReLU / Eq. 9: A2B chain (R9) or one-round FSS (R22)")
     ap.add_argument("--no-classes", action="store_true",
                     help="skip the CUPTI kernel-class leg (required under ncu: one CUPTI client at a time)")
     ap.add_argument("--task", default="mlp", choices=sorted(WORKLOADS),
@@ -400,7 +404,8 @@ def bench_split(args):
     cap = (96 << 20) if TASK == "cnn" else (8 << 20)
     xp = make_transport(party, peer, kind=os.environ.get("PSML_XPORT", "peer"), capacity_bytes=cap)
     dp = make_dp(list(range(party * half, (party + 1) * half)), rank, groups[party])
-    tr = PartyTrainer(TASK, synth.init_weights(TASK), party, xp, batch=BATCH, pair_id=pair, dp=dp)
+    tr = PartyTrainer(TASK, synth.init_weights(TASK), party, xp, batch=BATCH, pair_id=pair, dp=dp,
+                      mask_reuse=args.mask_reuse, compare=args.compare)
     nb = min(K + W, 64)
     Xs, Ys, Xh, Yh = [], [], [], []
     for s in range(nb):
@@ -464,7 +469,8 @@ def bench_split(args):
         "config": {"workload": WORKLOAD, "deployment": "split (party 0 on GPU k, party 1 on GPU k + N/2)",
                    "global_batch": BATCH * half, "per_pair_batch": BATCH, "pairs": half,
                    "ring": "Z_2^64, 13 fractional bits", "parallelism": f"{half} pairs x 2 parties",
-                   "transport": xp_kind(), "l2": "256 MiB flush between timed steps (outside the events)",
+                   "transport": xp_kind(), "mask_reuse": bool(args.mask_reuse), "compare": args.compare,
+                   "l2": "256 MiB flush between timed steps (outside the events)",
                    "step": "client share, dealer of the next step (forked graph branch), online step "
                            "with one exchange per opening round, per-party gradient all-reduce, update: "
                            "one CUDA graph per party"},
