@@ -53,6 +53,7 @@ def parse():
                     help="split deployment: SecureML forward/backward mask reuse (DESIGN.md R26)")
     ap.add_argument("--compare", default="a2b", choices=["a2b", "fss"],
                     help="secure comparison of ReLU / Eq. 9: A2B chain (R9) or one-round FSS (R22)")
+    ap.add_argument("--no-secondary", action="store_true", help="skip the other configs' figures")
     ap.add_argument("--no-classes", action="store_true",
                     help="skip the CUPTI kernel-class leg (required under ncu: one CUPTI client at a time)")
     ap.add_argument("--task", default="mlp", choices=sorted(WORKLOADS),
@@ -885,16 +886,75 @@ def cpu_baseline(budget_s=12.0):
 # ---------------------------------------------------------------------------------------------
 # reference arm: the CPU oracle (oracle/protocol.py) on the same workload
 # ---------------------------------------------------------------------------------------------
-def oracle_steps(n_steps, base=0):
+def oracle_steps(n_steps, base=0, task=None):
     import synth
     from oracle import core
     from oracle import protocol as OP
-    m = OP.Model(TASK, synth.init_weights(TASK))
+    task = task or TASK
+    m = OP.Model(task, synth.init_weights(task))
     t0 = time.perf_counter()
     for s in range(n_steps):
-        X, Y = synth.batch(TASK, base + s)
+        X, Y = synth.batch(task, base + s)
         OP.train_step(m, X, Y, base + s)
     return time.perf_counter() - t0, core.num_threads()
+
+
+SECONDARY = (("linreg", "config 2: secure linear regression, MNIST-shaped, batch 128"),
+             ("logreg", "config 2: secure logistic regression (Eq. 9), MNIST-shaped, batch 128"),
+             ("cnn", "config 4: secure CNN (conv 5x5x16 im2col, FC 64, FC 10), CIFAR-shaped, batch 128"),
+             ("svm", "SURVEY f4: secure linear SVM (hinge subgradient, DESIGN.md R24), MNIST-shaped, batch 128"),
+             ("rnn", "SURVEY f4: secure Elman RNN (T = 16, BPTT, DESIGN.md R25), synthetic sequences, batch 128"))
+
+
+def secondary_figures(K=50):
+    """The other BASELINE configs / workloads on the same GPU, each as its own pipelined CUDA graph
+    (client share + next step's dealer + online step + update), K timed steps after a warm-up, CUDA
+    events with the 256 MiB L2 flush between steps; secure inference (forward half + its dealer);
+    beside the oracle timed on the host (a few whole steps; 1 for the CNN)."""
+    import torch
+    import synth
+    from paper_conf_icpp_chenzzzz020_b200.train import SecureTrainer
+    dev = torch.device("cuda")
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream()
+    out = {}
+    for task, what in SECONDARY:
+        try:
+            tr = SecureTrainer(task, synth.init_weights(task))
+            data = [synth.batch(task, s) for s in range(8)]
+            Xs = [torch.from_numpy(x).to(dev) for x, _ in data]
+            Ys = [torch.from_numpy(y).to(dev) for _, y in data]
+            tr.step(Xs[0], Ys[0], 0)
+            tr.capture(pipelined=True)
+
+            def timed(fn, n, base):
+                evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(n)]
+                torch.cuda.synchronize()
+                for i in range(n):
+                    flush.zero_()
+                    evs[i][0].record(stream)
+                    fn(base + i)
+                    evs[i][1].record(stream)
+                torch.cuda.synchronize()
+                return sum(a.elapsed_time(b) for a, b in evs) / 1e3
+            timed(lambda s: tr.graph_step(Xs[s % 8], Ys[s % 8], s), 3, 1)
+            n = K if task != "cnn" else max(10, K // 4)
+            t = timed(lambda s: tr.graph_step(Xs[s % 8], Ys[s % 8], s), n, 4)
+
+            def infer(s):
+                Xsh, _ = tr.share_batch(Xs[s % 8], Ys[s % 8], s)
+                tr.infer_shares(Xsh, s)
+            ti = timed(infer, n, 100000)
+            tr.close()
+            n_or = 1 if task == "cnn" else 5
+            t_or, cores = oracle_steps(n_or, base=20000, task=task)
+            out[task] = {"config": what, "samples_per_s": 128 * n / t, "ms_per_step": 1e3 * t / n,
+                         "infer_samples_per_s": 128 * n / ti, "steps": n,
+                         "cpu_baseline": {"value": 128 * n_or / t_or, "unit": "samples/s", "cores": cores,
+                                          "kind": "oracle", "sample": f"{n_or} whole oracle training step(s)"}}
+        except Exception as e:   # noqa: BLE001 -- reported, never fatal to the headline line
+            out[task] = {"config": what, "error": str(e)[:300]}
+    return out
 
 
 def arm_config(world):
@@ -960,6 +1020,8 @@ def main():
         result["beaver_matmul_cfg1"] = beaver_latency_figure()
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         result["cpu_baseline"] = cpu_baseline()
+    if rank == 0 and world == 1 and not args.no_secondary:
+        result["secondary_configs"] = secondary_figures()
     if rank == 0:
         print(json.dumps(result), flush=True)
 

@@ -9,9 +9,9 @@ timeout 900 python bench.py > gpurun_out/${T}_bench.json 2> gpurun_out/${T}_benc
 echo "bench rc=$?"; tail -c 1500 gpurun_out/${T}_bench.json; tail -3 gpurun_out/${T}_bench.err
 if [ "$2" != "nocu" ]; then
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 2000 --csv --log-file gpurun_out/${T}_launches.csv \
-  python bench.py --steps 20 --warmup 3 --no-ring-gemm --no-cpu-baseline --no-classes > /dev/null 2>&1; echo "ncu list rc=$?"
+  python bench.py --steps 20 --warmup 3 --no-ring-gemm --no-cpu-baseline --no-classes --no-secondary > /dev/null 2>&1; echo "ncu list rc=$?"
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:"seg_gemm|tc_seg|msb_chain|had_fused|open_list|deal_prg" \
-  -s 400 -c 12 -o gpurun_out/${T}_full python bench.py --steps 20 --warmup 3 --no-ring-gemm --no-cpu-baseline --no-classes > /dev/null 2>&1; echo "ncu full rc=$?"
+  -s 400 -c 12 -o gpurun_out/${T}_full python bench.py --steps 20 --warmup 3 --no-ring-gemm --no-cpu-baseline --no-classes --no-secondary > /dev/null 2>&1; echo "ncu full rc=$?"
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:"tc_ring|tc_finalize|split" -c 6 \
   -o gpurun_out/${T}_ring4096 python tools/ring_gemm_once.py 4096 64 1 > /dev/null 2>&1; echo "ncu ring rc=$?"
 fi
