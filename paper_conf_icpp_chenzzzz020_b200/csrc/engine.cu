@@ -504,20 +504,22 @@ psml_status psml_msb_dealer(psml_ring ring, uint64_t seed, uint64_t call_id, int
 // ------------------------------------------------------------------------------------------------
 // server side
 // ------------------------------------------------------------------------------------------------
-// Config 1 (one linear-regression minibatch, A M x K . B K x 1) in ONE launch: a warp per output
-// row, both parties.  Each warp re-derives the opened F = (B_0 - V_0) + (B_1 - V_1) of its K
-// columns (K words, L2-resident) and the opened row E_m = (A_0 - U_0) + (A_1 - U_1) (Eqs. 4-5),
-// then C_p[m] = p E_m.F + E_m.V_p + U_p[m].F + Z_p[m] (BJ form, the Eq. 8 K-concatenation), and
-// the SecureML truncation -- the mask, open and GEMV rounds of the co-resident pair fused.
+// Config 1 (one linear-regression minibatch, A M x K . B K x 1) in ONE launch: a CTA per output
+// row, both parties; its 8 warps split K.  Each thread re-derives the opened F = (B_0 - V_0) +
+// (B_1 - V_1) of its K columns (K words, L2-resident) and the opened row E_m = (A_0 - U_0) +
+// (A_1 - U_1) (Eqs. 4-5), accumulates p E_m.F + E_m.V_p + U_p[m].F (BJ form, the Eq. 8
+// K-concatenation), and the CTA adds Z_p[m] and truncates -- the mask, open and GEMV rounds of the
+// co-resident pair fused.
 template <typename T>
 __global__ void __launch_bounds__(256) beaver_gemv_kernel(CPair<T> A, CPair<T> B, CPair<T> U, CPair<T> V, CPair<T> Z,
                                                           int64_t M, int64_t K, int trunc, Pair<T> C) {
-    const int lane = threadIdx.x & 31;
-    const int64_t row = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    if (row >= M) return;
+    __shared__ T red[2][8];
+    const int64_t row = blockIdx.x;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     T acc0 = 0, acc1 = 0;
     const T *a0 = A.p[0] + row * K, *a1 = A.p[1] + row * K, *u0 = U.p[0] + row * K, *u1 = U.p[1] + row * K;
-    for (int64_t k = lane; k < K; k += 32) {
+#pragma unroll 2
+    for (int64_t k = tid; k < K; k += 256) {
         const T f = (B.p[0][k] - V.p[0][k]) + (B.p[1][k] - V.p[1][k]);
         const T uu0 = __ldcs(u0 + k), uu1 = __ldcs(u1 + k);
         const T e = (__ldcs(a0 + k) - uu0) + (__ldcs(a1 + k) - uu1);
@@ -529,9 +531,13 @@ __global__ void __launch_bounds__(256) beaver_gemv_kernel(CPair<T> A, CPair<T> B
         acc0 += __shfl_xor_sync(0xffffffffu, acc0, o);
         acc1 += __shfl_xor_sync(0xffffffffu, acc1, o);
     }
-    if (lane == 0) {
-        C.p[0][row] = trunc_share<T>(acc0 + Z.p[0][row], 0, trunc);
-        C.p[1][row] = trunc_share<T>(acc1 + Z.p[1][row], 1, trunc);
+    if (lane == 0) { red[0][warp] = acc0; red[1][warp] = acc1; }
+    __syncthreads();
+    if (tid < 2) {
+        T acc = 0;
+#pragma unroll
+        for (int w = 0; w < 8; ++w) acc += red[tid][w];
+        C.p[tid][row] = trunc_share<T>(acc + Z.p[tid][row], tid, trunc);
     }
 }
 
@@ -550,7 +556,7 @@ static psml_status secure_matmul_t(Ctx *c, const void *const A[2], const void *c
     }
     if (!tr && flags == 0 && N == 1 && K <= 65536) {   // config 1: one fused launch
         ProfScope prof(PROF_GEMM, s, (double)M * 2 * K * 2);
-        beaver_gemv_kernel<T><<<(unsigned)((M * 32 + 255) / 256), 256, 0, s>>>(
+        beaver_gemv_kernel<T><<<(unsigned)M, 256, 0, s>>>(
             CPair<T>{{a[0], a[1]}}, CPair<T>{{b[0], b[1]}}, CPair<T>{{u[0], u[1]}}, CPair<T>{{v[0], v[1]}},
             CPair<T>{{z[0], z[1]}}, M, K, trunc, Pair<T>{{cc[0], cc[1]}});
         PSML_LAUNCH_CHECK();

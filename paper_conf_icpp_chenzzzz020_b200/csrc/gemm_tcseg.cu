@@ -15,6 +15,9 @@
 // the partial tiles are summed through distributed shared memory, and each CTA runs the epilogue
 // (+ Z_p, truncation, store) on 1/ks of the tile.  Ring addition is exact, so the result is
 // bit-identical to the CUDA-core seg_gemm_kernel (tested).
+#ifndef PSML_TCSEG_FILL
+#define PSML_TCSEG_FILL 2
+#endif
 #include <cooperative_groups.h>
 
 #include "engine.h"
@@ -520,9 +523,9 @@ psml_status tc_seg_group(const SegArgs<uint64_t> *jobs, int njobs, cudaStream_t 
 #ifdef TCSEG_TIMING
     if (const char *e = getenv("PSML_TCSEG_MMAS")) g.debug_mmas = atoi(e);
 #endif
-    // K split: double ks while the grid stays within half the SMs (the rest stays with the
-    // dealer branch) and each split keeps >= 2 K blocks
-    const int fill = 2;
+    // K split: double ks while the grid stays within 1/PSML_TCSEG_FILL of the SMs (default 2: the
+    // rest stays with the dealer branch) and each split keeps >= 2 K blocks
+    const int fill = PSML_TCSEG_FILL;
     int ks = 1;
     while (ks < max_ks && tiles * ks * 2 * fill <= 2 * sm_count && nkb_max >= ks * 2) ks *= 2;
     g.ks = ks;
