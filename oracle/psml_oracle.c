@@ -304,29 +304,73 @@ EXPORT void or_truncate(int l, int party, uint64_t *x, int64_t n, int d) {
 /*   daBit: rB_i = PRG('R','0'+i) & 1; rA_0 = PRG('R','A'); rA_1 = (rB_0 ^ rB_1) - rA_0.        */
 /* Material layout per party (uint64 words): [t][3][n] for (a,b,c) then rB[n], rA[n].           */
 /* ------------------------------------------------------------------------------------------ */
-static int log2_l(int l) { int L = 0; while ((1 << L) < l) ++L; return L; }
 
-EXPORT int64_t or_msb_material_words(int l, int64_t n) { return (int64_t)(2 * log2_l(l) * 3 + 2) * n; }
+/*
+ * Secure MSB by a REDUCED Kogge-Stone carry prefix (R27, replacing the full-word R9
+ * chain).  Only G[l-2] -- the carry into bit l-1 -- is needed, so after the first level only every
+ * other prefix position matters, then every fourth, ...: level 1 gates the even bit positions
+ * 2..l-2, after which the even positions are compacted into an l/2-bit word; every later level
+ * gates the odd positions of the current word (G at every odd index, P at odd indices >= 3) and
+ * compacts the odd positions.  For l = 64: 63 + 62 + 31 + 15 + 7 + 3 + 1 = 182 bit-ANDs instead of
+ * 12 x 64, in the same 1 + log2(l) rounds.  Each AND is a boolean Beaver AND restricted to its gate
+ * mask M: open e = (x ^ a) & M, f = (y ^ b) & M -- no bit outside M leaves a party.
+ *
+ * Material per element and party: 3 groups x (a, b, c) words + the daBit (r^B, r^A) = 11 words
+ * (structure of arrays: word w of element e at mat[w * n + e]; group g at words 3g .. 3g + 2):
+ *   group 0  round 0 (G = X0 & X1):  bits 0 .. l-2
+ *   group 1  level 1: the G gates at their own (even) positions, the P gates shifted down by 1
+ *            (odd positions): bits 1 .. l-2
+ *   group 2  levels 2 .. log2(l): level j occupies a field of w_j = l / 2^(j-1) bits at offset
+ *            sum of the previous widths; inside it the G gates at the odd positions and the P gates
+ *            shifted down by 1 (even positions): field bits 1 .. w_j - 1
+ * a_i = PRG('a', '0' + i, g) & mask_g, b_i likewise, c_0 = PRG('c', '0', g) & mask_g,
+ * c_1 = ((a_0 ^ a_1) & (b_0 ^ b_1)) ^ c_0; r^B_i = PRG('R', '0' + i) & 1, r^A_0 = PRG('R', 'A'),
+ * r^A_1 = (r^B_0 ^ r^B_1) - r^A_0.
+ */
+EXPORT int64_t or_msb_material_words(int l, int64_t n) { (void)l; return 11 * n; }
+
+static uint64_t bits_mask(int lo, int hi) {   /* bits lo .. hi inclusive (hi < 64) */
+    uint64_t m = 0;
+    for (int b = lo; b <= hi; ++b) m |= (uint64_t)1 << b;
+    return m;
+}
+
+static uint64_t msb_group_mask(int l, int g) {
+    if (g == 0) return bits_mask(0, l - 2);
+    if (g == 1) return bits_mask(1, l - 2);
+    uint64_t m = 0;
+    int off = 0;
+    for (int w = l / 2; w >= 2; w /= 2) {
+        m |= bits_mask(off + 1, off + w - 1);
+        off += w;
+    }
+    return m;
+}
 
 EXPORT void or_msb_dealer(int l, uint64_t seed, uint64_t call_id, int64_t n, uint64_t *mat0,
                           uint64_t *mat1) {
     uint64_t m = ring_mask(l);
-    int L = log2_l(l);
     uint64_t *mat[2] = {mat0, mat1};
-    for (int t = 0; t < 2 * L; ++t) {
+    for (int g = 0; g < 3; ++g) {
+        uint64_t gm = msb_group_mask(l, g);
         for (int i = 0; i < 2; ++i) {
-            dprg(l, seed, TAG('a', '0' + i, t, 0), call_id, 0, n, mat[i] + ((int64_t)t * 3 + 0) * n);
-            dprg(l, seed, TAG('b', '0' + i, t, 0), call_id, 0, n, mat[i] + ((int64_t)t * 3 + 1) * n);
+            dprg(64, seed, TAG('a', '0' + i, g, 0), call_id, 0, n, mat[i] + ((int64_t)g * 3 + 0) * n);
+            dprg(64, seed, TAG('b', '0' + i, g, 0), call_id, 0, n, mat[i] + ((int64_t)g * 3 + 1) * n);
         }
-        uint64_t *c0 = mat0 + ((int64_t)t * 3 + 2) * n, *c1 = mat1 + ((int64_t)t * 3 + 2) * n;
-        dprg(l, seed, TAG('c', '0', t, 0), call_id, 0, n, c0);
+        uint64_t *c0 = mat0 + ((int64_t)g * 3 + 2) * n, *c1 = mat1 + ((int64_t)g * 3 + 2) * n;
+        dprg(64, seed, TAG('c', '0', g, 0), call_id, 0, n, c0);
         for (int64_t e = 0; e < n; ++e) {
-            uint64_t a = mat0[((int64_t)t * 3 + 0) * n + e] ^ mat1[((int64_t)t * 3 + 0) * n + e];
-            uint64_t b = mat0[((int64_t)t * 3 + 1) * n + e] ^ mat1[((int64_t)t * 3 + 1) * n + e];
-            c1[e] = ((a & b) ^ c0[e]) & m;
+            for (int i = 0; i < 2; ++i) {
+                mat[i][((int64_t)g * 3 + 0) * n + e] &= gm;
+                mat[i][((int64_t)g * 3 + 1) * n + e] &= gm;
+            }
+            c0[e] &= gm;
+            uint64_t a = mat0[((int64_t)g * 3 + 0) * n + e] ^ mat1[((int64_t)g * 3 + 0) * n + e];
+            uint64_t b = mat0[((int64_t)g * 3 + 1) * n + e] ^ mat1[((int64_t)g * 3 + 1) * n + e];
+            c1[e] = (a & b) ^ c0[e];
         }
     }
-    int64_t off = (int64_t)2 * L * 3 * n;
+    int64_t off = 9 * n;
     dprg(l, seed, TAG('R', '0', 0, 0), call_id, 0, n, mat0 + off);
     dprg(l, seed, TAG('R', '1', 0, 0), call_id, 0, n, mat1 + off);
     for (int64_t e = 0; e < n; ++e) { mat0[off + e] &= 1; mat1[off + e] &= 1; }
@@ -335,75 +379,98 @@ EXPORT void or_msb_dealer(int l, uint64_t seed, uint64_t call_id, int64_t n, uin
         mat1[off + n + e] = ((mat0[off + e] ^ mat1[off + e]) - mat0[off + n + e]) & m;
 }
 
-/* One boolean Beaver AND for both parties on word vectors (GMW with a triplet):
- * open e = x ^ a, f = y ^ b; z_i = (i ? e&f : 0) ^ (e & b_i) ^ (a_i & f) ^ c_i. */
-static void bool_and(int64_t n, const uint64_t *x0, const uint64_t *x1, const uint64_t *y0,
-                     const uint64_t *y1, const uint64_t *a0, const uint64_t *a1, const uint64_t *b0,
-                     const uint64_t *b1, const uint64_t *c0, const uint64_t *c1, uint64_t *z0,
-                     uint64_t *z1) {
-    for (int64_t t = 0; t < n; ++t) {
-        uint64_t e = (x0[t] ^ a0[t]) ^ (x1[t] ^ a1[t]);
-        uint64_t f = (y0[t] ^ b0[t]) ^ (y1[t] ^ b1[t]);
-        uint64_t r0 = (e & b0[t]) ^ (a0[t] & f) ^ c0[t];
-        uint64_t r1 = (e & f) ^ (e & b1[t]) ^ (a1[t] & f) ^ c1[t];
-        z0[t] = r0; z1[t] = r1;
-    }
+/* One boolean Beaver AND for both parties of one element, restricted to the gate mask M:
+ * open e = (x ^ a) & M, f = (y ^ b) & M; z_i = (i ? e&f : 0) ^ (e & b_i) ^ (a_i & f) ^ c_i. */
+static void bool_and1(uint64_t M, uint64_t x0, uint64_t x1, uint64_t y0, uint64_t y1, uint64_t a0,
+                      uint64_t a1, uint64_t b0, uint64_t b1, uint64_t c0, uint64_t c1, uint64_t *z0,
+                      uint64_t *z1) {
+    uint64_t e = ((x0 ^ a0) & M) ^ ((x1 ^ a1) & M);
+    uint64_t f = ((y0 ^ b0) & M) ^ ((y1 ^ b1) & M);
+    *z0 = (e & b0) ^ (a0 & f) ^ c0;
+    *z1 = (e & f) ^ (e & b1) ^ (a1 & f) ^ c1;
+}
+
+/* Keep the bits at positions start, start + 2, start + 4, ... of a w-bit word, packed downwards. */
+static uint64_t compact(uint64_t v, int w, int start) {
+    uint64_t r = 0;
+    int k = 0;
+    for (int b = start; b < w; b += 2, ++k) r |= ((v >> b) & 1) << k;
+    return r;
+}
+
+static uint64_t odd_bits(int lo, int w) {   /* odd positions >= lo below w */
+    uint64_t m = 0;
+    for (int b = 1; b < w; b += 2)
+        if (b >= lo) m |= (uint64_t)1 << b;
+    return m;
 }
 
 /*
- * MSB of x = x_0 + x_1 mod 2^l, Kogge-Stone carry prefix on boolean shares.
- * P0 holds X0 := x_0 shared as (x_0, 0); P1 holds X1 := x_1 shared as (0, x_1).
- * G = X0 & X1 (AND t=0); P = X0 ^ X1 (local).  For level j = 1..L, k = 2^(j-1):
- *   G <- G ^ (P & (G << k))   (AND t = 2j-1)
- *   P <- P & (P << k)         (AND t = 2j, skipped at j = L)
- * msb = P_orig[l-1] ^ G[l-2].  Then B2A with the daBit: open c = msb ^ rB,
- * [msb]^A_i = (i==0 ? c : 0) + (1 - 2c) rA_i.   Output: arithmetic shares of msb (0/1).
- * Optional output: boolean shares of msb (bit 0 of a word).
+ * MSB of x = x_0 + x_1 mod 2^l on boolean shares (P0 holds X0 := x_0 as (x_0, 0), P1 holds
+ * X1 := x_1 as (0, x_1)), the reduced prefix of the header comment; msb = P_orig[l-1] ^ G[l-2].
+ * Then B2A with the daBit: open c = msb ^ rB, [msb]^A_i = (i==0 ? c : 0) + (1 - 2c) rA_i.
+ * Output: arithmetic shares of msb (0/1); optional boolean shares of msb (bit 0 of a word).
  */
 EXPORT void or_secure_msb(int l, const uint64_t *x0, const uint64_t *x1, int64_t n,
                           const uint64_t *mat0, const uint64_t *mat1, uint64_t *msbA0,
                           uint64_t *msbA1, uint64_t *msbB0, uint64_t *msbB1) {
     uint64_t m = ring_mask(l);
-    int L = log2_l(l);
-    size_t sz = sizeof(uint64_t) * n;
-    uint64_t *X0s0 = calloc(n, sizeof(uint64_t)), *X0s1 = calloc(n, sizeof(uint64_t));
-    uint64_t *X1s0 = calloc(n, sizeof(uint64_t)), *X1s1 = calloc(n, sizeof(uint64_t));
-    uint64_t *G0 = malloc(sz), *G1 = malloc(sz), *P0 = malloc(sz), *P1 = malloc(sz);
-    uint64_t *S0 = malloc(sz), *S1 = malloc(sz), *T0 = malloc(sz), *T1 = malloc(sz);
-    for (int64_t t = 0; t < n; ++t) { X0s0[t] = x0[t] & m; X1s1[t] = x1[t] & m; }
-#define MAT(i, tt, w) ((i) == 0 ? mat0 : mat1) + ((int64_t)(tt) * 3 + (w)) * n
-    bool_and(n, X0s0, X0s1, X1s0, X1s1, MAT(0, 0, 0), MAT(1, 0, 0), MAT(0, 0, 1), MAT(1, 0, 1),
-             MAT(0, 0, 2), MAT(1, 0, 2), G0, G1);
-    for (int64_t t = 0; t < n; ++t) { P0[t] = X0s0[t] ^ X1s0[t]; P1[t] = X0s1[t] ^ X1s1[t]; }
-    for (int j = 1; j <= L; ++j) {
-        int k = 1 << (j - 1);
-        for (int64_t t = 0; t < n; ++t) { S0[t] = (G0[t] << k) & m; S1[t] = (G1[t] << k) & m; }
-        bool_and(n, P0, P1, S0, S1, MAT(0, 2 * j - 1, 0), MAT(1, 2 * j - 1, 0), MAT(0, 2 * j - 1, 1),
-                 MAT(1, 2 * j - 1, 1), MAT(0, 2 * j - 1, 2), MAT(1, 2 * j - 1, 2), T0, T1);
-        if (j < L) {
-            for (int64_t t = 0; t < n; ++t) { S0[t] = (P0[t] << k) & m; S1[t] = (P1[t] << k) & m; }
-            uint64_t *Q0 = malloc(sz), *Q1 = malloc(sz);
-            bool_and(n, P0, P1, S0, S1, MAT(0, 2 * j, 0), MAT(1, 2 * j, 0), MAT(0, 2 * j, 1),
-                     MAT(1, 2 * j, 1), MAT(0, 2 * j, 2), MAT(1, 2 * j, 2), Q0, Q1);
-            memcpy(P0, Q0, sz); memcpy(P1, Q1, sz);
-            free(Q0); free(Q1);
-        }
-        for (int64_t t = 0; t < n; ++t) { G0[t] ^= T0[t]; G1[t] ^= T1[t]; }
-    }
-#undef MAT
-    int64_t off = (int64_t)2 * L * 3 * n;
     for (int64_t t = 0; t < n; ++t) {
-        uint64_t b0 = ((X0s0[t] >> (l - 1)) & 1) ^ ((G0[t] >> (l - 2)) & 1); /* P_orig share 0 = x_0 */
-        uint64_t b1 = ((X1s1[t] >> (l - 1)) & 1) ^ ((G1[t] >> (l - 2)) & 1); /* P_orig share 1 = x_1 */
+#define W(i, g, k) ((i) == 0 ? mat0 : mat1)[((int64_t)(g) * 3 + (k)) * n + t]
+        uint64_t X0 = x0[t] & m, X1 = x1[t] & m;
+        uint64_t G[2], P[2];
+        /* round 0: G = X0 & X1 on bits 0 .. l-2; P = X0 ^ X1 (local) */
+        bool_and1(bits_mask(0, l - 2), X0, 0, 0, X1, W(0, 0, 0), W(1, 0, 0), W(0, 0, 1), W(1, 0, 1),
+                  W(0, 0, 2), W(1, 0, 2), &G[0], &G[1]);
+        P[0] = X0; P[1] = X1;
+        /* level 1 (shift 1): gates at the even positions 2 .. l-2; the group-1 word carries the
+         * G material there and the P material shifted down by one */
+        {
+            uint64_t MG = 0;
+            for (int b = 2; b <= l - 2; b += 2) MG |= (uint64_t)1 << b;
+            uint64_t zG[2], zP[2], aG[2], bG[2], cG[2], aP[2], bP[2], cP[2];
+            for (int i = 0; i < 2; ++i) {
+                aG[i] = W(i, 1, 0) & MG; aP[i] = (W(i, 1, 0) << 1) & MG;
+                bG[i] = W(i, 1, 1) & MG; bP[i] = (W(i, 1, 1) << 1) & MG;
+                cG[i] = W(i, 1, 2) & MG; cP[i] = (W(i, 1, 2) << 1) & MG;
+            }
+            bool_and1(MG, P[0], P[1], G[0] << 1, G[1] << 1, aG[0], aG[1], bG[0], bG[1], cG[0], cG[1], &zG[0], &zG[1]);
+            bool_and1(MG, P[0], P[1], P[0] << 1, P[1] << 1, aP[0], aP[1], bP[0], bP[1], cP[0], cP[1], &zP[0], &zP[1]);
+            for (int i = 0; i < 2; ++i) {
+                G[i] = compact(G[i] ^ zG[i], l, 0);
+                P[i] = compact(zP[i], l, 0);
+            }
+        }
+        /* levels 2 .. log2(l) on the compacted words: gates at the odd positions (P at >= 3) */
+        int off = 0;
+        for (int w = l / 2; w >= 2; w /= 2) {
+            uint64_t MG = odd_bits(1, w), MP = odd_bits(3, w), fm = (w == 64) ? ~(uint64_t)0 : (((uint64_t)1 << w) - 1);
+            uint64_t zG[2], zP[2], aG[2], bG[2], cG[2], aP[2], bP[2], cP[2];
+            for (int i = 0; i < 2; ++i) {
+                uint64_t A = (W(i, 2, 0) >> off) & fm, Bw = (W(i, 2, 1) >> off) & fm, Cw = (W(i, 2, 2) >> off) & fm;
+                aG[i] = A & MG; aP[i] = (A << 1) & MP;
+                bG[i] = Bw & MG; bP[i] = (Bw << 1) & MP;
+                cG[i] = Cw & MG; cP[i] = (Cw << 1) & MP;
+            }
+            bool_and1(MG, P[0], P[1], G[0] << 1, G[1] << 1, aG[0], aG[1], bG[0], bG[1], cG[0], cG[1], &zG[0], &zG[1]);
+            bool_and1(MP, P[0], P[1], P[0] << 1, P[1] << 1, aP[0], aP[1], bP[0], bP[1], cP[0], cP[1], &zP[0], &zP[1]);
+            for (int i = 0; i < 2; ++i) {
+                G[i] = compact(G[i] ^ zG[i], w, 1);
+                P[i] = compact(zP[i], w, 1);
+            }
+            off += w;
+        }
+#undef W
+        uint64_t b0 = ((X0 >> (l - 1)) & 1) ^ (G[0] & 1); /* P_orig share 0 = x_0 */
+        uint64_t b1 = ((X1 >> (l - 1)) & 1) ^ (G[1] & 1); /* P_orig share 1 = x_1 */
         if (msbB0) msbB0[t] = b0;
         if (msbB1) msbB1[t] = b1;
-        uint64_t c = (b0 ^ mat0[off + t]) ^ (b1 ^ mat1[off + t]); /* B2A opening */
+        int64_t doff = 9 * n;
+        uint64_t c = (b0 ^ mat0[doff + t]) ^ (b1 ^ mat1[doff + t]); /* B2A opening */
         uint64_t s = (1 - 2 * c) & m;
-        msbA0[t] = (c + s * mat0[off + n + t]) & m;
-        msbA1[t] = (s * mat1[off + n + t]) & m;
+        msbA0[t] = (c + s * mat0[doff + n + t]) & m;
+        msbA1[t] = (s * mat1[doff + n + t]) & m;
     }
-    free(X0s0); free(X0s1); free(X1s0); free(X1s1);
-    free(G0); free(G1); free(P0); free(P1); free(S0); free(S1); free(T0); free(T1);
 }
 
 /* ------------------------------------------------------------------------------------------ */

@@ -219,6 +219,29 @@ def test_secure_msb_l64_edges(orc):
     assert [int(v) for v in orc.reconstruct(a0, a1)] == [bf.msb(v, 64) for v in vals]
 
 
+@pytest.mark.parametrize("l,gates", [(64, 182), (32, 87), (16, 40), (8, 17)])
+def test_reduced_msb_material_layout(orc, l, gates):
+    """R27: 11 material words per element and party; the AND material occupies exactly the gate
+    bits of the reduced prefix (l = 64: 63 + 2*31 + 31 + 15 + 7 + 3 + 1 = 182 of 12 x 64 full-word
+    AND bits), nothing outside them, and every group is a valid boolean triplet."""
+    n = 4096
+    assert orc.lib().or_msb_material_words(l, n) == 11 * n
+    m0, m1 = orc.msb_dealer(SEED + 2, 77, n, l)
+    union = 0
+    for g in range(3):
+        a = m0[(3 * g) * n:(3 * g + 1) * n] ^ m1[(3 * g) * n:(3 * g + 1) * n]
+        b = m0[(3 * g + 1) * n:(3 * g + 2) * n] ^ m1[(3 * g + 1) * n:(3 * g + 2) * n]
+        c = m0[(3 * g + 2) * n:(3 * g + 3) * n] ^ m1[(3 * g + 2) * n:(3 * g + 3) * n]
+        assert np.array_equal(c, a & b)
+        seen = 0
+        for w in (a, b, m0[(3 * g) * n:(3 * g + 1) * n]):
+            for v in w.tolist():
+                seen |= v
+        union += bin(seen).count("1")
+    assert union == gates   # 4096 random words light up every gate bit and nothing else
+    assert set(np.unique(m0[9 * n:10 * n]).tolist()) <= {0, 1}
+
+
 def test_secure_relu_and_eq9_exhaustive_l16(orc):
     l, f = 16, 4
     n = 1 << l
@@ -272,6 +295,8 @@ def test_dealer_key_separation(orc):
         assert orc.stream_seed(seed, orc.tag(bytes([ord("c"), ord("0"), t]))) == s0
     m0, m1 = orc.msb_dealer(seed, 5, 64)
     n = 64
-    # party 1's a/b words from s_1 alone; its c words are derived (need a_0, b_0 too)
-    assert np.array_equal(m1[:n], orc.prg(64, s1, orc.tag(bytes([ord("a"), ord("1"), 0])), 5, n))
+    # party 1's a/b words from s_1 alone (masked to the round-0 gate bits 0..62, R27); its c words
+    # are derived (need a_0, b_0 too)
+    mask0 = np.uint64((1 << 63) - 1)
+    assert np.array_equal(m1[:n], orc.prg(64, s1, orc.tag(bytes([ord("a"), ord("1"), 0])), 5, n) & mask0)
     assert not np.array_equal(m1[2 * n:3 * n], orc.prg(64, s1, orc.tag(bytes([ord("c"), ord("1"), 0])), 5, n))
