@@ -19,6 +19,7 @@ enum { PJ_SINGLE = 0, PJ_PAIR = 1, PJ_HAD = 2, PJ_AND = 3, PJ_DABIT = 4 };
 
 struct PrgJob {
     int kind;
+    uint64_t mask;        // PJ_AND: the group's gate bits (reduced prefix, R27)
     uint32_t tag[5];
     uint64_t cid;         // call id with step field 0
     int64_t n;            // elements
@@ -106,6 +107,30 @@ __global__ void __launch_bounds__(128, PSML_DEAL_MINB) deal_prg_kernel(const Prg
             deal_store8(J.out[3], e0, n, x);
             continue;
         }
+        if (kind == PJ_AND) {   // a0 a1 b0 b1 c0 -> c1 = ((a0^a1)&(b0^b1))^c0, every word masked
+            const uint64_t mk = J.mask;
+#pragma unroll
+            for (int j = 0; j < 8; ++j) { v[j] &= mk; x[j] = v[j]; }
+            deal_store8(J.out[0], e0, n, v);
+            deal_block(dkey(S, J.tag[1], cid), (uint32_t)b, v);
+#pragma unroll
+            for (int j = 0; j < 8; ++j) { v[j] &= mk; x[j] ^= v[j]; }
+            deal_store8(J.out[1], e0, n, v);
+            deal_block(dkey(S, J.tag[2], cid), (uint32_t)b, y);
+#pragma unroll
+            for (int j = 0; j < 8; ++j) y[j] &= mk;
+            deal_store8(J.out[2], e0, n, y);
+            deal_block(dkey(S, J.tag[3], cid), (uint32_t)b, v);
+#pragma unroll
+            for (int j = 0; j < 8; ++j) { v[j] &= mk; x[j] &= y[j] ^ v[j]; }
+            deal_store8(J.out[3], e0, n, v);
+            deal_block(dkey(S, J.tag[4], cid), (uint32_t)b, v);
+#pragma unroll
+            for (int j = 0; j < 8; ++j) { v[j] &= mk; x[j] ^= v[j]; }
+            deal_store8(J.out[4], e0, n, v);
+            deal_store8(J.out[5], e0, n, x);
+            continue;
+        }
         deal_store8(J.out[0], e0, n, v);
         if (kind == PJ_SINGLE) continue;
 #pragma unroll
@@ -113,8 +138,7 @@ __global__ void __launch_bounds__(128, PSML_DEAL_MINB) deal_prg_kernel(const Prg
         deal_block(dkey(S, J.tag[1], cid), (uint32_t)b, v);
         deal_store8(J.out[1], e0, n, v);
         if (kind == PJ_PAIR) continue;
-        if (kind == PJ_HAD) deal_tail<true>(J, S, cid, (uint32_t)b, e0, n, x, v);
-        else deal_tail<false>(J, S, cid, (uint32_t)b, e0, n, x, v);
+        deal_tail<true>(J, S, cid, (uint32_t)b, e0, n, x, v);   // PJ_HAD
     }
 }
 

@@ -486,7 +486,7 @@ psml_status psml_hadamard_triplet_gen(psml_ring ring, uint64_t seed, uint64_t ca
 
 int64_t psml_msb_material_words(psml_ring ring, int64_t n) {
     if (ring.l != 32 && ring.l != 64) return -1;
-    return (int64_t)(6 * ilog2_int(ring.l) + 2) * n;
+    return (int64_t)MSB_WORDS * n;   // reduced prefix material (R27)
 }
 
 psml_status psml_msb_dealer(psml_ring ring, uint64_t seed, uint64_t call_id, int64_t n, void *const mat[2],

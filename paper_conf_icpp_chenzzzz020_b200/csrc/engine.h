@@ -56,7 +56,7 @@ psml_status msb_dealer_launch(const DealSeeds &S, uint64_t cid, int64_t n, void 
                               const uint32_t *step = nullptr) {
     const int L = ilog2_int(8 * (int)sizeof(T));
     const int64_t nblk = (n + PerBlock<T>::value - 1) / PerBlock<T>::value;
-    dim3 grid((unsigned)grid_for(nblk, 128, 148 * 8), (unsigned)(2 * L + 1));
+    dim3 grid((unsigned)grid_for(nblk, 128, 148 * 8), 4u);   // 3 AND groups + the daBit (R27)
     msb_dealer_kernel<T><<<grid, 128, 0, s>>>(S, cid, n, L, (T *)mat[0], (T *)mat[1], step);
     PSML_LAUNCH_CHECK();
     return PSML_OK;

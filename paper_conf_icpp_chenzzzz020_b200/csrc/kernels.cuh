@@ -174,44 +174,68 @@ __global__ void hadamard_triplet_kernel(PrgKey ku0, PrgKey ku1, PrgKey kv0, PrgK
     }
 }
 
-// MSB material: blockIdx.y = AND index t (0 .. 2L-1) or 2L for the daBit.
+// MSB material of the reduced prefix (R27): blockIdx.y = group g (0 .. 2) or 3 for the
+// daBit.  Group g's a / b / c words are masked to its gate bits (msb_group_mask).
+__host__ __device__ inline uint64_t low_bits(int w) { return w >= 64 ? ~(uint64_t)0 : (((uint64_t)1 << w) - 1); }
+__host__ __device__ inline uint64_t msb_group_mask(int l, int g) {
+    if (g == 0) return low_bits(l - 1);                    // round 0: bits 0 .. l-2
+    if (g == 1) return low_bits(l - 1) & ~(uint64_t)1;     // level 1: bits 1 .. l-2
+    uint64_t m = 0;                                        // levels 2..: fields of l/2, l/4, ... bits
+    int off = 0;
+    for (int w = l / 2; w >= 2; w /= 2) {
+        m |= (low_bits(w) & ~(uint64_t)1) << off;
+        off += w;
+    }
+    return m;
+}
+constexpr int MSB_WORDS = 11;   // 3 groups x (a, b, c) + daBit (r^B, r^A), per element and party
+
 template <typename T>
 __global__ void msb_dealer_kernel(const DealSeeds S, uint64_t call_id, int64_t n, int L, T *__restrict__ m0,
                                   T *__restrict__ m1, const uint32_t *step) {
-    constexpr int PB = PerBlock<T>::value;
+    constexpr int PB = PerBlock<uint64_t>::value;
+    constexpr int l = 8 * (int)sizeof(T);
+    (void)L;
     if (step) {
         const uint64_t st = *step;
         call_id = (call_id & ~(0xFFFFFFFFull << 24)) | (st << 24);
     }
-    const int t = blockIdx.y;
+    const int g = blockIdx.y;
     const int64_t nblk = (n + PB - 1) / PB;
+    const uint64_t gm = g < 3 ? msb_group_mask(l, g) : 0;
     for (int64_t b = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; b < nblk; b += (int64_t)gridDim.x * blockDim.x) {
-        if (t < 2 * L) {
+        if (g < 3) {
             uint32_t wa0[16], wa1[16], wb0[16], wb1[16], wc0[16];
-            chacha20_block(dkey(S, tag4('a', '0', t), call_id), (uint32_t)b, wa0);
-            chacha20_block(dkey(S, tag4('a', '1', t), call_id), (uint32_t)b, wa1);
-            chacha20_block(dkey(S, tag4('b', '0', t), call_id), (uint32_t)b, wb0);
-            chacha20_block(dkey(S, tag4('b', '1', t), call_id), (uint32_t)b, wb1);
-            chacha20_block(dkey(S, tag4('c', '0', t), call_id), (uint32_t)b, wc0);
-            T *base0 = m0 + (int64_t)t * 3 * n, *base1 = m1 + (int64_t)t * 3 * n;
+            chacha20_block(dkey(S, tag4('a', '0', g), call_id), (uint32_t)b, wa0);
+            chacha20_block(dkey(S, tag4('a', '1', g), call_id), (uint32_t)b, wa1);
+            chacha20_block(dkey(S, tag4('b', '0', g), call_id), (uint32_t)b, wb0);
+            chacha20_block(dkey(S, tag4('b', '1', g), call_id), (uint32_t)b, wb1);
+            chacha20_block(dkey(S, tag4('c', '0', g), call_id), (uint32_t)b, wc0);
+            T *base0 = m0 + (int64_t)g * 3 * n, *base1 = m1 + (int64_t)g * 3 * n;
 #pragma unroll
             for (int j = 0; j < PB; ++j) {
                 int64_t e = b * PB + j;
                 if (e >= n) break;
-                T a0 = word_of<T>(wa0, j), a1 = word_of<T>(wa1, j), b0 = word_of<T>(wb0, j);
-                T b1 = word_of<T>(wb1, j), c0 = word_of<T>(wc0, j);
-                base0[e] = a0; base0[n + e] = b0; base0[2 * n + e] = c0;
-                base1[e] = a1; base1[n + e] = b1; base1[2 * n + e] = ((a0 ^ a1) & (b0 ^ b1)) ^ c0;
+                const uint64_t a0 = word_of<uint64_t>(wa0, j) & gm, a1 = word_of<uint64_t>(wa1, j) & gm;
+                const uint64_t b0 = word_of<uint64_t>(wb0, j) & gm, b1 = word_of<uint64_t>(wb1, j) & gm;
+                const uint64_t c0 = word_of<uint64_t>(wc0, j) & gm;
+                base0[e] = (T)a0; base0[n + e] = (T)b0; base0[2 * n + e] = (T)c0;
+                base1[e] = (T)a1; base1[n + e] = (T)b1; base1[2 * n + e] = (T)(((a0 ^ a1) & (b0 ^ b1)) ^ c0);
             }
-        } else {
+        }
+    }
+    if (g == 3) {   // daBit: r^B_i = PRG(R, i) & 1 (l-bit stream), r^A_0 = PRG(R, A), r^A_1 = r - r^A_0
+        constexpr int PBT = PerBlock<T>::value;
+        const int64_t nbt = (n + PBT - 1) / PBT;
+        for (int64_t b = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; b < nbt; b += (int64_t)gridDim.x * blockDim.x) {
             uint32_t w0[16], w1[16], wa[16];
             chacha20_block(dkey(S, TAG_R0, call_id), (uint32_t)b, w0);
             chacha20_block(dkey(S, TAG_R1, call_id), (uint32_t)b, w1);
             chacha20_block(dkey(S, TAG_RA, call_id), (uint32_t)b, wa);
-            const int64_t off = (int64_t)2 * L * 3 * n;
+            const int64_t off = (int64_t)9 * n;
 #pragma unroll
-            for (int j = 0; j < PB; ++j) {
-                int64_t e = b * PB + j;
+            for (int j = 0; j < PBT; ++j) {
+                int64_t e = b * PBT + j;
                 if (e >= n) break;
                 T r0 = word_of<T>(w0, j) & 1, r1 = word_of<T>(w1, j) & 1, ra0 = word_of<T>(wa, j);
                 m0[off + e] = r0; m1[off + e] = r1;
@@ -315,82 +339,132 @@ __device__ __forceinline__ T msb_input(const MsbArgs<T> &a, int p, int64_t e) {
 }
 
 template <typename T>
-__device__ __forceinline__ const T *mat_ptr(const MsbArgs<T> &a, int p, int t, int w) {
-    return a.mat.p[p] + ((int64_t)t * 3 + w) * a.n;
+__device__ __forceinline__ const T *mat_ptr(const MsbArgs<T> &a, int p, int g, int w) {
+    return a.mat.p[p] + ((int64_t)g * 3 + w) * a.n;
 }
 
-// open one AND (message words w, w+1) of AND index t: returns both parties' z.
-template <typename T>
-__device__ __forceinline__ void and_open(const MsbArgs<T> &a, int64_t e, int w, int t, T z[2]) {
-    const T ee = a.msg.p[0][(int64_t)w * a.n + e] ^ a.msg.p[1][(int64_t)w * a.n + e];
-    const T ff = a.msg.p[0][(int64_t)(w + 1) * a.n + e] ^ a.msg.p[1][(int64_t)(w + 1) * a.n + e];
-#pragma unroll
-    for (int p = 0; p < 2; ++p) {
-        PSML_PARTY_SKIP(a, p)
-        T r = (ee & mat_ptr(a, p, t, 1)[e]) ^ (mat_ptr(a, p, t, 0)[e] & ff) ^ mat_ptr(a, p, t, 2)[e];
-        z[p] = p == 1 ? (T)(r ^ (ee & ff)) : r;
+// ---- the reduced Kogge-Stone prefix (R27) ---------------------------------------------
+// Bit gather of positions start, start + 2, ... of v into the low bits (start 0: even, 1: odd).
+__device__ __forceinline__ uint64_t compact_bits(uint64_t x, int start) {
+    x = (x >> start) & 0x5555555555555555ull;
+    x = (x | (x >> 1)) & 0x3333333333333333ull;
+    x = (x | (x >> 2)) & 0x0F0F0F0F0F0F0F0Full;
+    x = (x | (x >> 4)) & 0x00FF00FF00FF00FFull;
+    x = (x | (x >> 8)) & 0x0000FFFF0000FFFFull;
+    x = (x | (x >> 16)) & 0x00000000FFFFFFFFull;
+    return x;
+}
+// Level j = 1 .. L of an l-bit prefix: word width w = l >> (j - 1); material group (1 for j = 1,
+// else 2 at field offset l - 2w); gate masks of the G and P ANDs.
+struct MsbLevel {
+    int w, group, off;
+    uint64_t MG, MP;
+};
+__device__ __forceinline__ MsbLevel msb_level(int l, int j) {
+    MsbLevel v;
+    v.w = l >> (j - 1);
+    if (j == 1) {   // even positions 2 .. l-2, both gates
+        v.group = 1; v.off = 0;
+        v.MG = v.MP = 0x5555555555555555ull & low_bits(l - 1) & ~(uint64_t)1;
+    } else {        // odd positions (P: >= 3) of the compacted w-bit word
+        v.group = 2; v.off = l - 2 * v.w;
+        v.MG = 0xAAAAAAAAAAAAAAAAull & low_bits(v.w);
+        v.MP = v.MG & ~(uint64_t)2;
     }
+    return v;
+}
+// unpack a group word into the level's G-gate and P-gate material (P stored shifted down by one)
+__device__ __forceinline__ void msb_unpack(const MsbLevel &v, uint64_t word, uint64_t &gpart, uint64_t &ppart) {
+    const uint64_t f = (word >> v.off) & low_bits(v.w);
+    gpart = f & v.MG;
+    ppart = (f << 1) & v.MP;
+}
+// one restricted boolean Beaver AND for party p: z_p = (p ? e&f : 0) ^ (e & b_p) ^ (a_p & f) ^ c_p
+__device__ __forceinline__ uint64_t and_z(int p, uint64_t e, uint64_t f, uint64_t a, uint64_t b, uint64_t c) {
+    const uint64_t r = (e & b) ^ (a & f) ^ c;
+    return p == 1 ? (r ^ (e & f)) : r;
 }
 
 // ---- per-element round bodies (one protocol round each) -----------------------------------------
-// Round 1: mask AND t = 0 with X = (x0, 0), Y = (0, x1).
+// Round 1: mask AND 0 (G = X0 & X1 on bits 0 .. l-2) with X = (x0, 0), Y = (0, x1).
 template <typename T>
 __device__ __forceinline__ void msb_round0_body(const MsbArgs<T> &a, int64_t e) {
+    const uint64_t M0 = low_bits(a.l - 1);
 #pragma unroll
     for (int p = 0; p < 2; ++p) {
         PSML_PARTY_SKIP(a, p)
-        T x = msb_input(a, p, e);
-        T X = p == 0 ? x : (T)0, Y = p == 1 ? x : (T)0;
-        a.msg.p[p][e] = X ^ mat_ptr(a, p, 0, 0)[e];
-        a.msg.p[p][a.n + e] = Y ^ mat_ptr(a, p, 0, 1)[e];
+        const uint64_t x = (uint64_t)msb_input(a, p, e);
+        const uint64_t X = p == 0 ? x : 0, Y = p == 1 ? x : 0;
+        a.msg.p[p][e] = (T)((X ^ (uint64_t)mat_ptr(a, p, 0, 0)[e]) & M0);
+        a.msg.p[p][a.n + e] = (T)((Y ^ (uint64_t)mat_ptr(a, p, 0, 1)[e]) & M0);
     }
 }
 
-// Round j+1 (j = 1..L): open level j-1's ANDs, update G/P, mask level j's ANDs.
+// open the AND of level jp (0 = round 0) from message words 0, 1: G / P of both parties, compacted
+template <typename T>
+__device__ __forceinline__ void msb_open_level(const MsbArgs<T> &a, int64_t e, int jp, uint64_t G[2], uint64_t P[2]) {
+    const uint64_t E = (uint64_t)a.msg.p[0][e] ^ (uint64_t)a.msg.p[1][e];
+    const uint64_t Fo = (uint64_t)a.msg.p[0][a.n + e] ^ (uint64_t)a.msg.p[1][a.n + e];
+    if (jp == 0) {
+#pragma unroll
+        for (int p = 0; p < 2; ++p) {
+            PSML_PARTY_SKIP(a, p)
+            G[p] = and_z(p, E, Fo, mat_ptr(a, p, 0, 0)[e], mat_ptr(a, p, 0, 1)[e], mat_ptr(a, p, 0, 2)[e]);
+            P[p] = (uint64_t)msb_input(a, p, e);
+        }
+        return;
+    }
+    const MsbLevel v = msb_level(a.l, jp);
+    uint64_t eG, eP, fG, fP;
+    msb_unpack(MsbLevel{v.w, v.group, 0, v.MG, v.MP}, E, eG, eP);   // messages are packed at offset 0
+    msb_unpack(MsbLevel{v.w, v.group, 0, v.MG, v.MP}, Fo, fG, fP);
+#pragma unroll
+    for (int p = 0; p < 2; ++p) {
+        PSML_PARTY_SKIP(a, p)
+        uint64_t aG, aP, bG, bP, cG, cP;
+        msb_unpack(v, mat_ptr(a, p, v.group, 0)[e], aG, aP);
+        msb_unpack(v, mat_ptr(a, p, v.group, 1)[e], bG, bP);
+        msb_unpack(v, mat_ptr(a, p, v.group, 2)[e], cG, cP);
+        const uint64_t zG = and_z(p, eG, fG, aG, bG, cG), zP = and_z(p, eP, fP, aP, bP, cP);
+        const int start = jp == 1 ? 0 : 1;
+        G[p] = compact_bits((uint64_t)a.G.p[p][e] ^ zG, start);
+        P[p] = compact_bits(zP, start);
+    }
+}
+
+// Round j+1 (j = 1..L): open level j-1's AND, mask level j's G and P ANDs (one packed word each).
 template <typename T>
 __device__ __forceinline__ void msb_level_body(const MsbArgs<T> &a, int j, int64_t e) {
-    const int k = 1 << (j - 1);
-    T G[2], P[2], z[2];
-    if (j == 1) {
-        and_open(a, e, 0, 0, z);
-#pragma unroll
-        for (int p = 0; p < 2; ++p) { PSML_PARTY_SKIP(a, p) G[p] = z[p]; P[p] = msb_input(a, p, e); }
-    } else {
-        and_open(a, e, 0, 2 * j - 3, z);
-        T zp[2];
-        and_open(a, e, 2, 2 * j - 2, zp);
-#pragma unroll
-        for (int p = 0; p < 2; ++p) { PSML_PARTY_SKIP(a, p) G[p] = a.G.p[p][e] ^ z[p]; P[p] = zp[p]; }
-    }
+    uint64_t G[2] = {0, 0}, P[2] = {0, 0};
+    msb_open_level(a, e, j - 1, G, P);
+    const MsbLevel v = msb_level(a.l, j);
 #pragma unroll
     for (int p = 0; p < 2; ++p) {
         PSML_PARTY_SKIP(a, p)
-        const int t1 = 2 * j - 1;
-        a.msg.p[p][e] = P[p] ^ mat_ptr(a, p, t1, 0)[e];
-        a.msg.p[p][a.n + e] = (T)(G[p] << k) ^ mat_ptr(a, p, t1, 1)[e];
-        if (j < a.L) {
-            const int t2 = 2 * j;
-            a.msg.p[p][2 * a.n + e] = P[p] ^ mat_ptr(a, p, t2, 0)[e];
-            a.msg.p[p][3 * a.n + e] = (T)(P[p] << k) ^ mat_ptr(a, p, t2, 1)[e];
-        }
-        a.G.p[p][e] = G[p];
-        a.P.p[p][e] = P[p];
+        uint64_t aG, aP, bG, bP;
+        msb_unpack(v, mat_ptr(a, p, v.group, 0)[e], aG, aP);
+        msb_unpack(v, mat_ptr(a, p, v.group, 1)[e], bG, bP);
+        const uint64_t eG = (P[p] ^ aG) & v.MG, fG = ((G[p] << 1) ^ bG) & v.MG;
+        const uint64_t eP = (P[p] ^ aP) & v.MP, fP = ((P[p] << 1) ^ bP) & v.MP;
+        a.msg.p[p][e] = (T)(eG | (eP >> 1));
+        a.msg.p[p][a.n + e] = (T)(fG | (fP >> 1));
+        a.G.p[p][e] = (T)G[p];
+        a.P.p[p][e] = (T)P[p];
     }
 }
 
-// Round L+2: open the last G AND, msb_i = x_i[l-1] ^ G_i[l-2]; emit the B2A message c_i.
+// Round L+2: open the last level's AND, msb_i = x_i[l-1] ^ G_i[l-2] (bit 0 of the compacted G);
+// emit the B2A message c_i.
 template <typename T>
 __device__ __forceinline__ void msb_final_body(const MsbArgs<T> &a, const Pair<T> &msbB, int64_t e) {
-    const int t = 2 * a.L - 1;
-    const int64_t off = (int64_t)2 * a.L * 3 * a.n;
-    T z[2];
-    and_open(a, e, 0, t, z);
+    const int64_t off = (int64_t)9 * a.n;
+    uint64_t G[2] = {0, 0}, P[2] = {0, 0};
+    msb_open_level(a, e, a.L, G, P);
 #pragma unroll
     for (int p = 0; p < 2; ++p) {
         PSML_PARTY_SKIP(a, p)
-        T G = a.G.p[p][e] ^ z[p];
-        T x = msb_input(a, p, e);
-        T b = ((x >> (a.l - 1)) & 1) ^ ((G >> (a.l - 2)) & 1);
+        const T x = msb_input(a, p, e);
+        const T b = ((x >> (a.l - 1)) & 1) ^ (T)(G[p] & 1);
         if (msbB.p[p]) msbB.p[p][e] = b;
         a.msg.p[p][e] = b ^ a.mat.p[p][off + e];   // c_i = msb_i ^ rB_i
     }
@@ -402,7 +476,7 @@ template <typename T>
 __device__ __forceinline__ void msb_b2a_body(const MsbArgs<T> &a, const Pair<T> &msbA, const Pair<T> &drelu,
                                              const CPair<T> &U, const CPair<T> &V, const Pair<T> &mE,
                                              const Pair<T> &mF, int what, int64_t e) {
-    const int64_t off = (int64_t)2 * a.L * 3 * a.n;
+    const int64_t off = (int64_t)9 * a.n;
     const T c = a.msg.p[0][e] ^ a.msg.p[1][e];
     const T s = (T)1 - (T)2 * c;
 #pragma unroll
@@ -590,12 +664,12 @@ __global__ void __launch_bounds__(256) msb_chain_pair_kernel(MsbArgs<T> a, Chain
     // written by a kernel that completed before any PDL predecessor of this one could start (the
     // previous graph's dealer, or a dealer launch without early trigger), so it is loaded BEFORE
     // griddepcontrol.wait, overlapping the predecessor's tail; only x depends on the predecessor.
-    T mt[2 * L][3];
+    uint64_t mt[3][3];   // the reduced prefix's material (R27): 3 groups x (a, b, c)
 #pragma unroll
-    for (int t = 0; t < 2 * L; ++t)
+    for (int g = 0; g < 3; ++g)
 #pragma unroll
-        for (int w = 0; w < 3; ++w) mt[t][w] = mat[((int64_t)t * 3 + w) * n + e];
-    const int64_t off = (int64_t)2 * L * 3 * n;
+        for (int w = 0; w < 3; ++w) mt[g][w] = (uint64_t)mat[((int64_t)g * 3 + w) * n + e];
+    const int64_t off = (int64_t)9 * n;
     const T rB = mat[off + e], rA = mat[off + n + e];
     T hu = 0, hv = 0, hz = 0, ysub = 0;
     if (MODE != 0) { hu = SEL(o.U)[e]; hv = SEL(o.V)[e]; hz = SEL(o.Z)[e]; }
@@ -625,27 +699,29 @@ __global__ void __launch_bounds__(256) msb_chain_pair_kernel(MsbArgs<T> a, Chain
             }
         }
     };
-    auto M = [&](int t, int w) -> T { return mt[t][w]; };
-    auto z_of = [&](T ee, T ff, int t) -> T {
-        T r = (ee & M(t, 1)) ^ (M(t, 0) & ff) ^ M(t, 2);
-        return p == 1 ? (T)(r ^ (ee & ff)) : r;
-    };
-    // round 1: AND t = 0 on X = (x0, 0), Y = (0, x1)
-    T m0 = (p == 0 ? x : (T)0) ^ M(0, 0), m1 = (p == 1 ? x : (T)0) ^ M(0, 1);
-    T G = z_of(m0 ^ peer_of(m0), m1 ^ peer_of(m1), 0);
-    T P = x;
+    // round 1: AND 0 on X = (x0, 0), Y = (0, x1), bits 0 .. l-2
+    const uint64_t M0 = low_bits(l - 1), xw = (uint64_t)x;
+    const uint64_t m0 = ((p == 0 ? xw : 0) ^ mt[0][0]) & M0, m1 = ((p == 1 ? xw : 0) ^ mt[0][1]) & M0;
+    uint64_t G = and_z(p, m0 ^ peer_of(m0), m1 ^ peer_of(m1), mt[0][0], mt[0][1], mt[0][2]);
+    uint64_t P = xw;
 #pragma unroll
-    for (int j = 1; j <= L; ++j) {
-        const int k = 1 << (j - 1);
-        const int t1 = 2 * j - 1, t2 = 2 * j;
-        const T g1 = P ^ M(t1, 0), h1 = (T)(G << k) ^ M(t1, 1);
-        T g2 = 0, h2 = 0;
-        if (j < L) { g2 = P ^ M(t2, 0); h2 = (T)(P << k) ^ M(t2, 1); }
-        const T z1 = z_of(g1 ^ peer_of(g1), h1 ^ peer_of(h1), t1);
-        if (j < L) P = z_of(g2 ^ peer_of(g2), h2 ^ peer_of(h2), t2);
-        G ^= z1;
+    for (int j = 1; j <= L; ++j) {   // one round per level: the packed G and P ANDs
+        const MsbLevel v = msb_level(l, j);
+        uint64_t aG, aP, bG, bP, cG, cP;
+        msb_unpack(v, mt[v.group][0], aG, aP);
+        msb_unpack(v, mt[v.group][1], bG, bP);
+        msb_unpack(v, mt[v.group][2], cG, cP);
+        const uint64_t eG = (P ^ aG) & v.MG, fG = ((G << 1) ^ bG) & v.MG;
+        const uint64_t eP = (P ^ aP) & v.MP, fP = ((P << 1) ^ bP) & v.MP;
+        const uint64_t me = eG | (eP >> 1), mf = fG | (fP >> 1);   // this party's two message words
+        const uint64_t E = me ^ peer_of(me), Fo = mf ^ peer_of(mf);
+        const uint64_t oG = E & v.MG, oP = (E << 1) & v.MP, qG = Fo & v.MG, qP = (Fo << 1) & v.MP;
+        const uint64_t zG = and_z(p, oG, qG, aG, bG, cG), zP = and_z(p, oP, qP, aP, bP, cP);
+        const int start = j == 1 ? 0 : 1;
+        G = compact_bits(G ^ zG, start);
+        P = compact_bits(zP, start);
     }
-    const T bit = ((x >> (l - 1)) & 1) ^ ((G >> (l - 2)) & 1);
+    const T bit = ((x >> (l - 1)) & 1) ^ (T)(G & 1);
     if (valid && SEL(o.msbB)) SEL(o.msbB)[e] = bit;
     const T cm = bit ^ rB;                    // B2A: c_i = msb_i ^ rB_i
     const T c = cm ^ peer_of(cm);

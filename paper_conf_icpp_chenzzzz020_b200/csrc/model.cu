@@ -490,6 +490,7 @@ static psml_status build_plan(psml_model_s *m, int pool, bool infer_only) {
         if (n <= 0) return;
         PrgJob j{};
         j.kind = kind;
+        j.mask = ~(uint64_t)0;
         int i = 0;
         for (uint32_t t : tags) j.tag[i++] = t;
         i = 0;
@@ -498,7 +499,6 @@ static psml_status build_plan(psml_model_s *m, int pool, bool infer_only) {
         P.chacha_blocks += (double)((n + 7) / 8) * (double)tags.size();
         (kind == PJ_PAIR || kind == PJ_SINGLE ? pjm : pjr).push_back(j);
     };
-    const int L = 6;   // log2(64): 2L AND triplets + one daBit per element (R9)
     auto &items = m->items[pool];
     for (size_t k = 0; k < items.size(); ++k) {
         DealItem &it = items[k];
@@ -529,15 +529,16 @@ static psml_status build_plan(psml_model_s *m, int pool, bool infer_only) {
             job(PJ_HAD, {TAG_U0, TAG_U1, TAG_V0, TAG_V1, TAG_Z0}, cid, it.n,
                 {it.U.p[0], it.U.p[1], it.V.p[0], it.V.p[1], it.Z.p[0], it.Z.p[1]});
             break;
-        case IT_MSB: {
+        case IT_MSB: {   // the reduced prefix's 3 AND groups + the daBit (R27)
             T *m0 = it.mat.p[0], *m1 = it.mat.p[1];
             const int64_t n = it.n;
-            for (int t = 0; t < 2 * L; ++t) {
-                const int64_t o = (int64_t)t * 3 * n;
-                job(PJ_AND, {tag4('a', '0', t), tag4('a', '1', t), tag4('b', '0', t), tag4('b', '1', t), tag4('c', '0', t)},
+            for (int g = 0; g < 3; ++g) {
+                const int64_t o = (int64_t)g * 3 * n;
+                job(PJ_AND, {tag4('a', '0', g), tag4('a', '1', g), tag4('b', '0', g), tag4('b', '1', g), tag4('c', '0', g)},
                     cid, n, {m0 + o, m1 + o, m0 + o + n, m1 + o + n, m0 + o + 2 * n, m1 + o + 2 * n});
+                pjr.back().mask = msb_group_mask(64, g);
             }
-            const int64_t o = (int64_t)2 * L * 3 * n;
+            const int64_t o = (int64_t)9 * n;
             job(PJ_DABIT, {TAG_R0, TAG_R1, TAG_RA}, cid, n, {m0 + o, m1 + o, m0 + o + n, m1 + o + n});
             break;
         }
@@ -1349,7 +1350,7 @@ static psml_status party_chain(PartyRun &r, const T *x, const DealItem *mat, con
             msb_level_kernel<T><<<g, EW_THREADS, 0, r.s>>>(a, j);
             PSML_LAUNCH_CHECK();
         }
-        PSML_TRY(xchg(r, {{snd, rcv, j < a.L ? 4 * n : 2 * n}}));
+        PSML_TRY(xchg(r, {{snd, rcv, 2 * n}}));   // the level's packed G and P AND messages (R27)
     }
     Pair<T> none{{nullptr, nullptr}};
     Pair<T> mE{{a.msg.p[0] + n, a.msg.p[1] + n}}, mF{{a.msg.p[0] + 2 * n, a.msg.p[1] + 2 * n}};
@@ -1741,7 +1742,6 @@ psml_status psml_model_deal(psml_model m, uint32_t step_id, int32_t infer_only, 
 // Words of party `party`'s material that its own seed cannot produce, in plan order (R23).
 static std::vector<std::pair<T *, int64_t>> derived_regions(psml_model_s *m, int pool, int party) {
     std::vector<std::pair<T *, int64_t>> r;
-    const int L = 6;   // log2(64): 2L AND triplets per MSB element
     for (auto &it : m->items[pool]) {
         switch (it.kind) {
         case IT_MATRIX:
@@ -1751,9 +1751,9 @@ static std::vector<std::pair<T *, int64_t>> derived_regions(psml_model_s *m, int
             if (party == 1) r.push_back({it.Z.p[1], it.Z.n});                 // Z_1 = U V - Z_0
             break;
         case IT_MSB:
-            if (party == 1) {
-                for (int t = 0; t < 2 * L; ++t) r.push_back({it.mat.p[1] + (3 * (int64_t)t + 2) * it.n, it.n});   // c_1
-                r.push_back({it.mat.p[1] + (6 * (int64_t)L + 1) * it.n, it.n});                                 // r^A_1
+            if (party == 1) {   // c_1 of the 3 AND groups, r^A_1 of the daBit (R27 layout)
+                for (int g = 0; g < 3; ++g) r.push_back({it.mat.p[1] + (3 * (int64_t)g + 2) * it.n, it.n});
+                r.push_back({it.mat.p[1] + 10 * it.n, it.n});
             }
             break;
         case IT_FSS:
