@@ -146,13 +146,16 @@ psml_status psml_triplet_gen(psml_ctx ctx, uint64_t seed, uint64_t call_id, int6
 psml_status psml_hadamard_triplet_gen(psml_ring ring, uint64_t seed, uint64_t call_id, int64_t n,
                                       void *const U[2], void *const V[2], void *const Z[2],
                                       psml_stream stream);
-/* Words (of l bits) of MSB material per party for n elements: (6 log2(l) + 2) n. */
+/* Words (of l bits) of MSB material per party for n elements: 11 n (R27). */
 int64_t psml_msb_material_words(psml_ring ring, int64_t n);
-/* Boolean AND triplets for the Kogge-Stone MSB and the daBit for B2A (R9).
- * mat[i] layout (words): for AND t = 0 .. 2 log2(l) - 1: a_i[n], b_i[n], c_i[n]; then
- * rB_i[n] (bit), rA_i[n].  a_i = PRG('a','0'+i,t), b_i = PRG('b','0'+i,t), c_0 = PRG('c','0',t),
- * c_1 = ((a_0^a_1) & (b_0^b_1)) ^ c_0; rB_i = PRG('R','0'+i) & 1; rA_0 = PRG('R','A'),
- * rA_1 = (rB_0 ^ rB_1) - rA_0. */
+/* Boolean AND triplets of the REDUCED Kogge-Stone prefix and the daBit for B2A (R27).
+ * mat[i] layout (words, structure of arrays): for AND group g = 0, 1, 2: a_i[n], b_i[n], c_i[n]
+ * (group 0: round 0 on bits 0..l-2; group 1: level 1, G material at the even positions 2..l-2 and
+ * P material shifted down by one; group 2: levels 2..log2(l), level j in a field of l/2^(j-1) bits
+ * at offset l - 2 l/2^(j-1), G material at its odd positions, P shifted down by one); then
+ * rB_i[n] (bit), rA_i[n].  a_i = PRG('a','0'+i,g) & mask_g, b_i = PRG('b','0'+i,g) & mask_g,
+ * c_0 = PRG('c','0',g) & mask_g, c_1 = ((a_0^a_1) & (b_0^b_1)) ^ c_0; rB_i = PRG('R','0'+i) & 1;
+ * rA_0 = PRG('R','A'), rA_1 = (rB_0 ^ rB_1) - rA_0.  Streams keyed per R23. */
 psml_status psml_msb_dealer(psml_ring ring, uint64_t seed, uint64_t call_id, int64_t n,
                             void *const mat[2], psml_stream stream);
 
@@ -208,8 +211,9 @@ psml_status psml_secure_hadamard(psml_ctx ctx, const void *const A[2], const voi
  * party 1: -((-x) >> bits) (logical shifts on l-bit values; R7). */
 psml_status psml_truncate(psml_ring ring, int32_t party, void *x_i, int64_t n, int32_t bits,
                           psml_stream stream);
-/* Arithmetic shares of MSB(x) (0/1) by Kogge-Stone A2B + daBit B2A: 1 + log2(l) rounds of
- * boolean ANDs then 1 B2A round.  mat from psml_msb_dealer.  msbB (nullable): boolean shares. */
+/* Arithmetic shares of MSB(x) (0/1) by the reduced Kogge-Stone A2B (R27: only the gate bits that
+ * reach the carry into bit l-1; 182 bit-ANDs at l = 64) + daBit B2A: 1 + log2(l) rounds of boolean
+ * ANDs then 1 B2A round.  mat from psml_msb_dealer.  msbB (nullable): boolean shares. */
 psml_status psml_secure_msb(psml_ctx ctx, const void *const x[2], int64_t n,
                             const void *const mat[2], void *const msbA[2], void *const msbB[2],
                             psml_stream stream);
