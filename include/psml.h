@@ -96,6 +96,30 @@ psml_status psml_bench_mac_peak(int32_t l, double *ring_macs_per_s);
 psml_status psml_ctx_create(psml_ring ring, int32_t gemm_backend, psml_ctx *out);
 psml_status psml_ctx_destroy(psml_ctx ctx);
 
+/* Execution options of a context (explicit arguments, no process globals).  Every field
+ * selects between bit-identical implementations (tested against each other and the oracle); the
+ * defaults are the measured fastest.  A call on a context -- or on a model created
+ * from it -- runs with that context's options.  psml_options_default fills the defaults. */
+typedef struct {
+    int32_t seg_backend;   /* training-step Beaver products: 0 auto (tcgen05 for groups of >= 2^25
+                              ring MACs on sm_100), 1 CUDA cores only, 2 tcgen05 wherever eligible */
+    int32_t pdl;           /* programmatic dependent launch between step kernels (1)          */
+    int32_t fused_open;    /* eager Beaver matmul: 0 mask round then GEMM (default), 1 mask fused
+                              into the GEMM's operand loads                                    */
+    int32_t fused_step;    /* co-resident MLP-family step: 1 producers open their consumers'
+                              operands (default), 0 one open pass per product                 */
+    int32_t fused_dealer;  /* 1 the step's dealer as two launches (default), 0 per item        */
+    int32_t deal_split;    /* pipelined graph: dealer PRG on two branches (1) or one (0)       */
+    int32_t deal_after;    /* pipelined graph: fork the dealer after this many online stages (1) */
+    int32_t gradw_branch;  /* weight gradients on their own graph branch (1)                  */
+    int32_t simt_cluster;  /* CUDA-core products: 1 cluster split-K kernel, 0 16 x 16 small tile */
+    int32_t rows_kernel;   /* CNN tall-skinny conv products: 1 rows kernel, 0 small tile        */
+    int32_t msb_chain;     /* MSB chain: 0 one lane-pair launch, 1 one kernel per round        */
+    int32_t conv_gw;       /* CNN weight gradient: 1 per-image kernel, 0 generic im2col GEMM    */
+} psml_options;
+psml_status psml_options_default(psml_options *out);
+psml_status psml_ctx_set_options(psml_ctx ctx, const psml_options *opts);
+
 /* ------------------------------------------------------------------------------------------ */
 /* PRG / client side (the client partitions inputs into shares)       */
 /* ------------------------------------------------------------------------------------------ */

@@ -102,6 +102,7 @@ using namespace psml;
 psml_status psml_delta_encode(psml_ctx ctx, const void *cur, const void *prev, int64_t rows, int64_t cols,
                               int32_t *row_ptr, int32_t *col_idx, void *vals, void *dense, int64_t *nnz_host,
                               int32_t *is_csr_host, psml_stream stream) {
+    PSML_CTX_OPTS(ctx);
     if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
     Ctx *c = reinterpret_cast<Ctx *>(ctx);
     if (rows <= 0 || cols <= 0 || rows * cols >= ((int64_t)1 << 31)) return fail(PSML_ERR_SHAPE, "bad rows/cols");
@@ -115,6 +116,7 @@ psml_status psml_delta_encode(psml_ctx ctx, const void *cur, const void *prev, i
 psml_status psml_delta_apply(psml_ctx ctx, int64_t rows, int64_t cols, int32_t is_csr, const int32_t *row_ptr,
                              const int32_t *col_idx, const void *vals, const void *dense, void *target,
                              psml_stream stream) {
+    PSML_CTX_OPTS(ctx);
     if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
     Ctx *c = reinterpret_cast<Ctx *>(ctx);
     if (rows <= 0 || cols <= 0) return fail(PSML_ERR_SHAPE, "bad rows/cols");

@@ -132,6 +132,15 @@ __host__ __device__ inline PrgKey make_key(uint64_t seed, uint32_t tag, uint64_t
     return k;
 }
 
+// The options of the context the current ABI call runs on (psml_options; a thread-local pointer
+// set for the duration of the call -- contexts are per host thread, include/psml.h).
+const psml_options &cur_opts();
+struct OptScope {
+    const psml_options *prev;
+    explicit OptScope(const psml_options *o);
+    ~OptScope();
+};
+
 // Dealer key separation (R23): each material stream is keyed by the seed of the party
 // that can produce it alone -- s_0 for U0 V0 Z0 a0 b0 c0 R0 RA F0 FS K0, s_1 for U1 V1 a1 b1 R1 K1 --
 // or by the dealer seed (the FSS input mask "FR").  s_i = PRG(dealer seed, "KD", i)[0].  A party that

@@ -270,6 +270,7 @@ psml_status psml_ctx_create_party(psml_ring ring, int32_t gemm_backend, int32_t 
 psml_status psml_secure_matmul_party(psml_ctx ctx, const void *A_i, const void *B_i, const void *U_i, const void *V_i,
                                      const void *Z_i, int64_t M, int64_t K, int64_t N, int32_t flags,
                                      int32_t trunc_bits, void *C_i, psml_stream stream) {
+    PSML_CTX_OPTS(ctx);
     if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
     Ctx *c = reinterpret_cast<Ctx *>(ctx);
     if (c->party < 0 || !c->xport) return fail(PSML_ERR_STATE, "not a per-party context (psml_ctx_create_party)");
@@ -287,6 +288,28 @@ psml_status psml_secure_matmul_party(psml_ctx ctx, const void *A_i, const void *
     const int64_t bytes[2] = {(int64_t)w * M * K, (int64_t)w * K * N};
     PSML_TRY(psml_xport_exchange(c->xport, 2, snd, rcv, bytes, stream));
     return psml_beaver_open_matmul(ctx, c->party, Es, Er, Fs, Fr, U_i, V_i, Z_i, M, K, N, trunc_bits, C_i, stream);
+}
+
+namespace psml {
+static const psml_options k_default_opts{0, 1, 0, 1, 1, 1, 1, 1, 1, 1, 0, 1};
+static thread_local const psml_options *t_opts = nullptr;
+const psml_options &cur_opts() { return t_opts ? *t_opts : k_default_opts; }
+OptScope::OptScope(const psml_options *o) : prev(t_opts) { if (o) t_opts = o; }
+OptScope::~OptScope() { t_opts = prev; }
+}  // namespace psml
+
+psml_status psml_options_default(psml_options *out) {
+    if (!out) return fail(PSML_ERR_INVALID, "out is null");
+    *out = k_default_opts;
+    return PSML_OK;
+}
+
+psml_status psml_ctx_set_options(psml_ctx ctx, const psml_options *o) {
+    if (!ctx || !o) return fail(PSML_ERR_INVALID, "null argument");
+    if (o->seg_backend < 0 || o->seg_backend > 2 || o->msb_chain < 0 || o->msb_chain > 1 || o->deal_after < 0)
+        return fail(PSML_ERR_INVALID, "option out of range");
+    reinterpret_cast<Ctx *>(ctx)->opts = *o;
+    return PSML_OK;
 }
 
 psml_status psml_ctx_destroy(psml_ctx ctx) {
@@ -461,6 +484,7 @@ static psml_status triplet_gen_t(Ctx *c, uint64_t seed, uint64_t cid, int64_t M,
 
 psml_status psml_triplet_gen(psml_ctx ctx, uint64_t seed, uint64_t call_id, int64_t M, int64_t K, int64_t N,
                              void *const U[2], void *const V[2], void *const Z[2], psml_stream stream) {
+    PSML_CTX_OPTS(ctx);
     if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
     Ctx *c = reinterpret_cast<Ctx *>(ctx);
     if (M <= 0 || K <= 0 || N <= 0) return fail(PSML_ERR_SHAPE, "M, K, N must be positive");
@@ -576,6 +600,7 @@ psml_status psml_secure_matmul(psml_ctx ctx, const void *const A[2], const void 
                                const void *const V[2], const void *const Z[2], int64_t M, int64_t K, int64_t N,
                                int32_t flags, int32_t trunc_bits, void *const C[2], const psml_trace *trace,
                                psml_stream stream) {
+    PSML_CTX_OPTS(ctx);
     if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
     Ctx *c = reinterpret_cast<Ctx *>(ctx);
     if (M <= 0 || K <= 0 || N <= 0) return fail(PSML_ERR_SHAPE, "M, K, N must be positive");
@@ -605,6 +630,7 @@ static psml_status beaver_mask_t(const void *A, const void *B, const void *U, co
 psml_status psml_beaver_mask(psml_ctx ctx, int32_t party, const void *A_i, const void *B_i, const void *U_i,
                              const void *V_i, int64_t M, int64_t K, int64_t N, int32_t flags, void *E_send,
                              void *F_send, psml_stream stream) {
+    PSML_CTX_OPTS(ctx);
     if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
     Ctx *c = reinterpret_cast<Ctx *>(ctx);
     if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
@@ -649,6 +675,7 @@ psml_status psml_beaver_open_matmul(psml_ctx ctx, int32_t party, const void *E_s
                                     const void *F_send, const void *F_recv, const void *U_i, const void *V_i,
                                     const void *Z_i, int64_t M, int64_t K, int64_t N, int32_t trunc_bits, void *C_i,
                                     psml_stream stream) {
+    PSML_CTX_OPTS(ctx);
     if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
     Ctx *c = reinterpret_cast<Ctx *>(ctx);
     if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
@@ -666,6 +693,7 @@ psml_status psml_beaver_open_matmul(psml_ctx ctx, int32_t party, const void *E_s
 psml_status psml_secure_hadamard(psml_ctx ctx, const void *const A[2], const void *const B[2], const void *const U[2],
                                  const void *const V[2], const void *const Z[2], int64_t n, int32_t trunc_bits,
                                  void *const C[2], psml_stream stream) {
+    PSML_CTX_OPTS(ctx);
     if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
     Ctx *c = reinterpret_cast<Ctx *>(ctx);
     if (n < 0) return fail(PSML_ERR_SHAPE, "n < 0");
@@ -714,6 +742,7 @@ static psml_status activation_t(Ctx *c, int what, const void *const x[2], int64_
 
 psml_status psml_secure_msb(psml_ctx ctx, const void *const x[2], int64_t n, const void *const mat[2],
                             void *const msbA[2], void *const msbB[2], psml_stream stream) {
+    PSML_CTX_OPTS(ctx);
     if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
     Ctx *c = reinterpret_cast<Ctx *>(ctx);
     if (n < 0) return fail(PSML_ERR_SHAPE, "n < 0");
@@ -728,6 +757,7 @@ psml_status psml_secure_msb(psml_ctx ctx, const void *const x[2], int64_t n, con
 psml_status psml_secure_relu(psml_ctx ctx, const void *const x[2], int64_t n, const void *const mat[2],
                              const void *const U[2], const void *const V[2], const void *const Z[2], void *const y[2],
                              void *const drelu[2], psml_stream stream) {
+    PSML_CTX_OPTS(ctx);
     if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
     Ctx *c = reinterpret_cast<Ctx *>(ctx);
     if (n < 0) return fail(PSML_ERR_SHAPE, "n < 0");
@@ -783,6 +813,7 @@ static psml_status fss_drelu_pair(const void *const x[2], int64_t n, const void 
 
 psml_status psml_secure_drelu_fss(psml_ctx ctx, const void *const x[2], int64_t n, const void *const mat[2],
                                   void *const drelu[2], void *xhat_trace, psml_stream stream) {
+    PSML_CTX_OPTS(ctx);
     if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
     Ctx *c = reinterpret_cast<Ctx *>(ctx);
     if (c->ring.l != 64) return fail(PSML_ERR_UNSUPPORTED, "the FSS comparison is built for Z_2^64");
@@ -798,6 +829,7 @@ psml_status psml_secure_drelu_fss(psml_ctx ctx, const void *const x[2], int64_t 
 psml_status psml_secure_relu_fss(psml_ctx ctx, const void *const x[2], int64_t n, const void *const mat[2],
                                  const void *const U[2], const void *const V[2], const void *const Z[2],
                                  void *const y[2], void *const drelu[2], psml_stream stream) {
+    PSML_CTX_OPTS(ctx);
     if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
     Ctx *c = reinterpret_cast<Ctx *>(ctx);
     if (c->ring.l != 64) return fail(PSML_ERR_UNSUPPORTED, "the FSS comparison is built for Z_2^64");
@@ -820,6 +852,7 @@ psml_status psml_secure_relu_fss(psml_ctx ctx, const void *const x[2], int64_t n
 // split deployment: party `party`'s round-1 message and its evaluation after the exchange
 psml_status psml_fss_mask(psml_ctx ctx, int32_t party, const void *x_i, int64_t n, const void *mat_i, void *msg,
                           psml_stream stream) {
+    PSML_CTX_OPTS(ctx);
     if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
     if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
     if (reinterpret_cast<Ctx *>(ctx)->ring.l != 64) return fail(PSML_ERR_UNSUPPORTED, "Z_2^64 only");
@@ -836,6 +869,7 @@ psml_status psml_fss_mask(psml_ctx ctx, int32_t party, const void *x_i, int64_t 
 
 psml_status psml_fss_open_drelu(psml_ctx ctx, int32_t party, const void *msg_send, const void *msg_recv, int64_t n,
                                 const void *mat_i, void *drelu_i, psml_stream stream) {
+    PSML_CTX_OPTS(ctx);
     if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
     if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
     if (reinterpret_cast<Ctx *>(ctx)->ring.l != 64) return fail(PSML_ERR_UNSUPPORTED, "Z_2^64 only");
@@ -871,6 +905,7 @@ static psml_status ring_gemm_t(Ctx *c, const void *A, const void *B, int64_t M, 
 
 psml_status psml_ring_gemm(psml_ctx ctx, const void *A, const void *B, int64_t M, int64_t K, int64_t N, void *C,
                            psml_stream stream) {
+    PSML_CTX_OPTS(ctx);
     if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
     Ctx *c = reinterpret_cast<Ctx *>(ctx);
     if (M <= 0 || K <= 0 || N <= 0) return fail(PSML_ERR_SHAPE, "M, K, N must be positive");

@@ -8,12 +8,15 @@
 namespace psml {
 
 psml_status check_ring(psml_ring r);
+// run the rest of an ABI call with the options of ctx / model (null: defaults)
+#define PSML_CTX_OPTS(c) ::psml::OptScope _psml_opts_((c) ? &reinterpret_cast<const ::psml::Ctx *>(c)->opts : nullptr)
 psml_status check_ptrs(std::initializer_list<const void *> ps);
 int current_sm_count();
 
 struct Ctx {
     psml_ring ring{64, 13};
     int backend = 0;    // 0 auto, 1 CUDA-core, 2 tcgen05
+    psml_options opts{0, 1, 0, 1, 1, 1, 1, 1, 1, 1, 0, 1};   // = psml_options_default
     int sm_count = 148;
     bool tc_ok = false;
     void *ws = nullptr;

@@ -605,26 +605,12 @@ __global__ void ring_gemm_finalize(Ops ops, const T *__restrict__ partial) {
 #include "gemm_seg.cuh"
 namespace psml {
 
-// PSML_SIMT=small: route small products to the 16 x 16 one-output-per-thread kernel instead of
-// the cluster split-K kernel (A/B switch; both bit-identical).
-inline bool simt_cl_enabled() {
-    static int v = -1;
-    if (v < 0) {
-        const char *e = getenv("PSML_SIMT");
-        v = (e && e[0] == 's') ? 0 : 1;
-    }
-    return v == 1;
-}
+// psml_options.simt_cluster = 0: route small products to the 16 x 16 one-output-per-thread kernel
+// instead of the cluster split-K kernel (both bit-identical).
+inline bool simt_cl_enabled() { return cur_opts().simt_cluster != 0; }
 
-// PSML_ROWS=0 keeps tall-skinny products on the 16 x 16 small-tile kernel.
-inline bool rows_kernel_enabled() {
-    static int v = -1;
-    if (v < 0) {
-        const char *e = getenv("PSML_ROWS");
-        v = (e && e[0] == '0') ? 0 : 1;
-    }
-    return v == 1;
-}
+// psml_options.rows_kernel = 0 keeps tall-skinny products on the 16 x 16 small-tile kernel.
+inline bool rows_kernel_enabled() { return cur_opts().rows_kernel != 0; }
 
 // ---------------------------------------------------------------------------------------------
 // host-side dispatcher: picks kernel, tile and split-K; `ws` must hold nparty*M*N words when

@@ -446,39 +446,23 @@ __global__ void __launch_bounds__(NT, 1) tc_seg_kernel(const __grid_constant__ G
 
 }  // namespace tcseg
 
-bool tc_seg_forced() {
-    static int v = -1;
-    if (v < 0) {
-        const char *e = getenv("PSML_SEG");
-        v = (e && e[0] == 't') ? 1 : 0;
-    }
-    return v == 1;
-}
+bool tc_seg_forced() { return cur_opts().seg_backend == 2; }   // psml_options.seg_backend
 
 bool tc_seg_enabled() {
-    static int v = -1;
-    if (v < 0) {
-        const char *e = getenv("PSML_SEG");
+    static int sm100 = -1;   // a device property, not an option
+    if (sm100 < 0) {
         int dev = 0, maj = 0, mnr = 0;
         cudaGetDevice(&dev);
         cudaDeviceGetAttribute(&maj, cudaDevAttrComputeCapabilityMajor, dev);
         cudaDeviceGetAttribute(&mnr, cudaDevAttrComputeCapabilityMinor, dev);
         cudaGetLastError();
-        // PSML_SEG=simt: CUDA-core two-segment GEMM; tcgen05 needs sm_100
-        v = (e && e[0] == 's') ? 0 : (maj == 10 && mnr == 0 ? 1 : 0);
+        sm100 = (maj == 10 && mnr == 0) ? 1 : 0;
     }
-    return v == 1;
+    return sm100 == 1 && cur_opts().seg_backend != 1;   // tcgen05 needs sm_100
 }
 
-// PSML_PDL=0 disables programmatic dependent launch of the GEMMs after their producer kernels.
-bool pdl_enabled() {
-    static int v = -1;
-    if (v < 0) {
-        const char *e = getenv("PSML_PDL");
-        v = (e && e[0] == '0') ? 0 : 1;
-    }
-    return v == 1;
-}
+// psml_options.pdl = 0 disables programmatic dependent launch of the GEMMs after their producers.
+bool pdl_enabled() { return cur_opts().pdl != 0; }
 
 psml_status tc_seg_group(const SegArgs<uint64_t> *jobs, int njobs, cudaStream_t stream, int sm_count) {
     using namespace tcseg;

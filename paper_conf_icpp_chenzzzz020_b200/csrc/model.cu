@@ -32,37 +32,16 @@ __global__ void set_word_kernel(uint32_t *p, uint32_t v) { *p = v; }
 
 // Co-resident Beaver matmuls run the explicit mask round then the GEMM that opens E/F (default:
 // measured faster inside the CUDA graph, 338K vs 328K samples/s) or fuse the mask into the GEMM's
-// operand loads (PSML_OPEN=fused: faster eagerly, one launch less); both bit-identical (tested).
-static bool fused_open() {
-    static int m = -1;
-    if (m < 0) {
-        const char *e = getenv("PSML_OPEN");
-        m = (e && e[0] == 'f') ? 1 : 0;
-    }
-    return m == 1;
-}
+// operand loads (psml_options.fused_open: faster eagerly, one launch less); bit-identical (tested).
+static bool fused_open() { return cur_opts().fused_open != 0; }
 
 // Fused co-resident training step (fused.cuh): producers open their consumers' operands
-// (default) or one open pass per product (PSML_FUSE=0); bit-identical (tested).
-static bool fuse_enabled() {
-    static int m = -1;
-    if (m < 0) {
-        const char *e = getenv("PSML_FUSE");
-        m = (e && e[0] == '0') ? 0 : 1;
-    }
-    return m == 1;
-}
+// (default) or one open pass per product (psml_options.fused_step = 0); bit-identical (tested).
+static bool fuse_enabled() { return cur_opts().fused_step != 0; }
 
 // The whole dealer of one step as two launches (dealer_fused.cuh; default) or one launch group per
-// item (PSML_DEAL=items); bit-identical (tested).
-static bool fused_deal() {
-    static int m = -1;
-    if (m < 0) {
-        const char *e = getenv("PSML_DEAL");
-        m = (e && e[0] == 'i') ? 0 : 1;
-    }
-    return m == 1;
-}
+// item (psml_options.fused_dealer = 0); bit-identical (tested).
+static bool fused_deal() { return cur_opts().fused_dealer != 0; }
 
 static inline uint64_t call_id(uint32_t pair, uint32_t step, int layer, int op, int slot) {
     return ((uint64_t)(pair & 0xFF) << 56) | ((uint64_t)step << 24) | ((uint64_t)(layer & 0xFF) << 16) |
@@ -573,15 +552,8 @@ static psml_status build_plan(psml_model_s *m, int pool, bool infer_only) {
     return PSML_OK;
 }
 
-// second dealer branch inside a pipelined capture (PSML_DEAL_SPLIT=0: one branch)
-static cudaStream_t deal_s2(psml_model_s *m) {
-    static int v = -1;
-    if (v < 0) {
-        const char *e = getenv("PSML_DEAL_SPLIT");
-        v = (e && e[0] == '0') ? 0 : 1;
-    }
-    return v ? m->side2 : nullptr;
-}
+// second dealer branch inside a pipelined capture (psml_options.deal_split = 0: one branch)
+static cudaStream_t deal_s2(psml_model_s *m) { return cur_opts().deal_split ? m->side2 : nullptr; }
 
 // PRG jobs [j0, j1) (blocks [b0, b1)) of plan P on stream s
 static psml_status deal_prg_launch(psml_model_s *m, const DealPlan &P, int j0, int j1, int64_t b0, int64_t b1,
@@ -979,14 +951,7 @@ static psml_status deal_fork_point(psml_model_s *m, cudaStream_t s, bool force =
 }
 
 
-static bool gradw_branch() {
-    static int v = -1;
-    if (v < 0) {
-        const char *e = getenv("PSML_GRADW_BRANCH");
-        v = (e && e[0] == '0') ? 0 : 1;
-    }
-    return v == 1;
-}
+static bool gradw_branch() { return cur_opts().gradw_branch != 0; }
 
 static psml_status fused_forward_backward(psml_model_s *m, const T *const X[2], const T *const Y[2], cudaStream_t s) {
     const int F = m->ctx->ring.frac_bits;
@@ -1498,6 +1463,7 @@ using namespace psml;
 // ABI definitions: C linkage and default visibility come from include/psml.h.
 
 psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_model *out) {
+    PSML_CTX_OPTS(ctx);
     if (!ctx || !desc || !out) return fail(PSML_ERR_INVALID, "null argument");
     Ctx *c = reinterpret_cast<Ctx *>(ctx);
     if (c->ring.l != 64) return fail(PSML_ERR_UNSUPPORTED, "training models run in Z_2^64 (DESIGN.md R18)");
@@ -1676,6 +1642,7 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
 }
 
 psml_status psml_model_destroy(psml_model model) {
+    PSML_CTX_OPTS(model ? model->ctx : nullptr);
     if (!model) return PSML_OK;
     cudaDeviceSynchronize();
     for (int g = 0; g < 2; ++g)
@@ -1698,6 +1665,7 @@ psml_status psml_model_destroy(psml_model model) {
 }
 
 psml_status psml_model_layer_shape(psml_model m, int32_t layer, int64_t *rows, int64_t *cols) {
+    PSML_CTX_OPTS(m ? m->ctx : nullptr);
     if (!m || layer < 0 || layer >= m->nl) return fail(PSML_ERR_INVALID, "bad model or layer");
     if (rows) *rows = m->rows[layer];
     if (cols) *cols = m->cols[layer];
@@ -1705,6 +1673,7 @@ psml_status psml_model_layer_shape(psml_model m, int32_t layer, int64_t *rows, i
 }
 
 psml_status psml_model_set_master(psml_model m, int32_t layer, const void *const Wm[2], psml_stream stream) {
+    PSML_CTX_OPTS(m ? m->ctx : nullptr);
     if (!m || layer < 0 || layer >= m->nl || !Wm) return fail(PSML_ERR_INVALID, "bad model, layer or pointer");
     PSML_TRY(check_ptrs({Wm[0], Wm[1]}));
     cudaStream_t s = (cudaStream_t)stream;
@@ -1719,6 +1688,7 @@ psml_status psml_model_set_master(psml_model m, int32_t layer, const void *const
 }
 
 psml_status psml_model_get_master(psml_model m, int32_t layer, void *const Wm[2], psml_stream stream) {
+    PSML_CTX_OPTS(m ? m->ctx : nullptr);
     if (!m || layer < 0 || layer >= m->nl || !Wm) return fail(PSML_ERR_INVALID, "bad model, layer or pointer");
     PSML_TRY(check_ptrs({Wm[0], Wm[1]}));
     const int64_t n = m->rows[layer] * m->cols[layer];
@@ -1728,6 +1698,7 @@ psml_status psml_model_get_master(psml_model m, int32_t layer, void *const Wm[2]
 }
 
 psml_status psml_model_deal(psml_model m, uint32_t step_id, int32_t infer_only, psml_stream stream) {
+    PSML_CTX_OPTS(m ? m->ctx : nullptr);
     if (!m) return fail(PSML_ERR_INVALID, "model is null");
     cudaStream_t s = (cudaStream_t)stream;
     const int pool = (int)(step_id & 1);
@@ -1766,6 +1737,7 @@ static std::vector<std::pair<T *, int64_t>> derived_regions(psml_model_s *m, int
 
 psml_status psml_model_deal_bundle(psml_model m, uint32_t step_id, int32_t party, void *bundle, int64_t *words,
                                    psml_stream stream) {
+    PSML_CTX_OPTS(m ? m->ctx : nullptr);
     if (!m || !words) return fail(PSML_ERR_INVALID, "null argument");
     if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
     if (m->d.deal_role != 0) return fail(PSML_ERR_STATE, "only the dealer (deal_role 0) writes bundles");
@@ -1787,6 +1759,7 @@ psml_status psml_model_deal_bundle(psml_model m, uint32_t step_id, int32_t party
 
 psml_status psml_model_deal_party(psml_model m, uint32_t step_id, int32_t party, const void *bundle, int64_t words,
                                   psml_stream stream) {
+    PSML_CTX_OPTS(m ? m->ctx : nullptr);
     if (!m) return fail(PSML_ERR_INVALID, "model is null");
     if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
     if (m->d.deal_role != party + 1) return fail(PSML_ERR_STATE, "model deal_role is not this party's");
@@ -1807,6 +1780,7 @@ psml_status psml_model_deal_party(psml_model m, uint32_t step_id, int32_t party,
 
 psml_status psml_train_forward_backward(psml_model m, const void *const X[2], const void *const Y[2], uint32_t step_id,
                                         psml_stream stream) {
+    PSML_CTX_OPTS(m ? m->ctx : nullptr);
     if (!m || !X || !Y) return fail(PSML_ERR_INVALID, "null argument");
     PSML_TRY(check_ptrs({X[0], X[1], Y[0], Y[1]}));
     const int pool = (int)(step_id & 1);
@@ -1821,6 +1795,7 @@ psml_status psml_train_forward_backward(psml_model m, const void *const X[2], co
 }
 
 psml_status psml_model_output(psml_model m, void **yhat0, void **yhat1, int64_t *n) {
+    PSML_CTX_OPTS(m ? m->ctx : nullptr);
     if (!m) return fail(PSML_ERR_INVALID, "model is null");
     if (yhat0) *yhat0 = m->yhat.p[0];
     if (yhat1) *yhat1 = m->yhat.p[1];
@@ -1829,6 +1804,7 @@ psml_status psml_model_output(psml_model m, void **yhat0, void **yhat1, int64_t 
 }
 
 psml_status psml_model_grads(psml_model m, void **grads, int64_t *words_per_party) {
+    PSML_CTX_OPTS(m ? m->ctx : nullptr);
     if (!m) return fail(PSML_ERR_INVALID, "model is null");
     if (grads) *grads = m->grad_base;
     if (words_per_party) *words_per_party = m->grad_words;
@@ -1836,6 +1812,7 @@ psml_status psml_model_grads(psml_model m, void **grads, int64_t *words_per_part
 }
 
 psml_status psml_train_apply_update(psml_model m, int32_t extra_shift, psml_stream stream) {
+    PSML_CTX_OPTS(m ? m->ctx : nullptr);
     if (!m) return fail(PSML_ERR_INVALID, "model is null");
     if (extra_shift < 0 || extra_shift > 16) return fail(PSML_ERR_INVALID, "extra_shift out of range");
     if (!m->grads_ready) return fail(PSML_ERR_STATE, "no gradients: run psml_train_forward_backward first");
@@ -1877,6 +1854,7 @@ psml_status psml_train_apply_update(psml_model m, int32_t extra_shift, psml_stre
 
 psml_status psml_secure_train_step(psml_model m, const void *const X[2], const void *const Y[2], uint32_t step_id,
                                    psml_stream stream) {
+    PSML_CTX_OPTS(m ? m->ctx : nullptr);
     PSML_TRY(psml_train_forward_backward(m, X, Y, step_id, stream));
     return psml_train_apply_update(m, 0, stream);
 }
@@ -1920,11 +1898,7 @@ static psml_status capture_one(psml_model_s *m, int pool, const T *const X[2], c
             if (cudaStreamWaitEvent(m->hi, m->ev_fork, 0) != cudaSuccess) st = fail(PSML_ERR_CUDA, "graph fork failed");
             on = m->hi;
         }
-        static int after = -1;
-        if (after < 0) {
-            const char *e = getenv("PSML_DEAL_AFTER");
-            after = e ? std::max(0, atoi(e)) : 1;   // after the step-start open (tools/gpu71.sh)
-        }
+        const int after = cur_opts().deal_after;   // default 1: after the step-start open
         // models without the fused step (the CNN) run large kernels that fill the GPU: their
         // dealer forks at the start of the step (measured: 51.6K vs 49.4K samples/s forked after)
         m->deal_after = (fused_eligible(m) && m->cap_party < 0) ? after : 0;
@@ -2012,6 +1986,7 @@ static psml_status capture_common(psml_model m, const void *const X[2], const vo
 
 psml_status psml_model_capture_step(psml_model m, const void *const X[2], const void *const Y[2], int32_t flags,
                                    psml_stream stream) {
+    PSML_CTX_OPTS(m ? m->ctx : nullptr);
     if (!m || !X || !Y) return fail(PSML_ERR_INVALID, "null argument");
     PSML_TRY(check_ptrs({X[0], X[1], Y[0], Y[1]}));
     m->cap_party = -1;
@@ -2022,6 +1997,7 @@ psml_status psml_model_capture_step(psml_model m, const void *const X[2], const 
 
 psml_status psml_party_capture_step(psml_model m, int32_t party, psml_xport x, psml_dp dp, const void *X_i,
                                     const void *Y_i, int32_t flags, psml_stream stream) {
+    PSML_CTX_OPTS(m ? m->ctx : nullptr);
     if (!m || !x) return fail(PSML_ERR_INVALID, "null model or transport");
     if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
     PSML_TRY(check_ptrs({X_i, Y_i}));
@@ -2081,6 +2057,7 @@ __global__ void copy_pair_kernel(const U *__restrict__ a, const U *__restrict__ 
 
 psml_status psml_model_step_host(psml_model m, const uint8_t *q, const void *y, int32_t y_kind, uint64_t share_seed,
                                  uint32_t step_id, void *yhat_host, psml_stream stream) {
+    PSML_CTX_OPTS(m ? m->ctx : nullptr);
     if (!m || !q || !y || !yhat_host) return fail(PSML_ERR_INVALID, "null argument");
     if (!m->graph[0] || !m->cap_X[0]) return fail(PSML_ERR_STATE, "no captured step: call psml_model_capture_step first");
     if (y_kind != 0 && y_kind != 1) return fail(PSML_ERR_INVALID, "y_kind: 0 float64 labels, 1 uint8 class indices");
@@ -2154,12 +2131,14 @@ psml_status psml_model_step_host(psml_model m, const uint8_t *q, const void *y, 
 }
 
 psml_status psml_model_graph_nodes(psml_model m, int64_t *n) {
+    PSML_CTX_OPTS(m ? m->ctx : nullptr);
     if (!m || !n) return fail(PSML_ERR_INVALID, "null argument");
     *n = m->graph_kernels + 1;   // + the step-word kernel launched before each replay
     return PSML_OK;
 }
 
 psml_status psml_model_step_graph(psml_model m, uint32_t step_id, psml_stream stream) {
+    PSML_CTX_OPTS(m ? m->ctx : nullptr);
     if (!m) return fail(PSML_ERR_INVALID, "model is null");
     if (!m->graph[0]) return fail(PSML_ERR_STATE, "no captured step: call psml_model_capture_step first");
     cudaStream_t s = (cudaStream_t)stream;
@@ -2192,6 +2171,7 @@ psml_status psml_model_step_graph(psml_model m, uint32_t step_id, psml_stream st
 
 psml_status psml_secure_infer(psml_model m, const void *const X[2], uint32_t step_id, void *const Yhat[2],
                               psml_stream stream) {
+    PSML_CTX_OPTS(m ? m->ctx : nullptr);
     if (!m || !X || !Yhat) return fail(PSML_ERR_INVALID, "null argument");
     PSML_TRY(check_ptrs({X[0], X[1], Yhat[0], Yhat[1]}));
     const int pool = (int)(step_id & 1);
@@ -2209,6 +2189,7 @@ psml_status psml_secure_infer(psml_model m, const void *const X[2], uint32_t ste
 // ------------------------------------------------------------------------------------------------
 psml_status psml_party_forward_backward(psml_model m, int32_t party, psml_xport x, const void *X_i, const void *Y_i,
                                         uint32_t step_id, psml_stream stream) {
+    PSML_CTX_OPTS(m ? m->ctx : nullptr);
     if (!m || !x) return fail(PSML_ERR_INVALID, "null model or transport");
     if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
     if (m->d.kind == PSML_SVM || m->d.kind == PSML_RNN)
@@ -2227,12 +2208,14 @@ psml_status psml_party_forward_backward(psml_model m, int32_t party, psml_xport 
 
 psml_status psml_party_train_step(psml_model m, int32_t party, psml_xport x, psml_dp dp, const void *X_i,
                                   const void *Y_i, uint32_t step_id, psml_stream stream) {
+    PSML_CTX_OPTS(m ? m->ctx : nullptr);
     PSML_TRY(psml_party_forward_backward(m, party, x, X_i, Y_i, step_id, stream));
     if (dp) PSML_TRY(dp_shift(dp).first);
     return party_reduce_update(m, party, dp, (cudaStream_t)stream);
 }
 
 psml_status psml_party_apply_update(psml_model m, int32_t party, int32_t extra_shift, psml_stream stream) {
+    PSML_CTX_OPTS(m ? m->ctx : nullptr);
     if (!m) return fail(PSML_ERR_INVALID, "model is null");
     if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
     if (extra_shift < 0 || extra_shift > 16) return fail(PSML_ERR_INVALID, "extra_shift out of range");

@@ -14,15 +14,8 @@ namespace psml {
 constexpr int EW_THREADS = 256;
 
 // MSB chain execution: 0 = one launch running each element through every round in order,
-// 1 = one kernel per round.  Environment override PSML_MSB_CHAIN=rounds (tests compare both).
-inline int chain_mode() {
-    static int m = -1;
-    if (m < 0) {
-        const char *e = getenv("PSML_MSB_CHAIN");
-        m = (e && e[0] == 'r') ? 1 : 0;
-    }
-    return m;
-}
+// 1 = one kernel per round (psml_options.msb_chain; tests compare both).
+inline int chain_mode() { return cur_opts().msb_chain; }
 
 inline int ew_grid(int64_t n) { return grid_for(n, EW_THREADS, 148 * 32); }
 
@@ -206,15 +199,8 @@ __global__ void __launch_bounds__(1024) conv_gw_image_kernel(const T *__restrict
     }
 }
 
-// PSML_CONV_GW=generic keeps the weight gradient on the generic im2col GEMM (tests)
-inline bool conv_gw_enabled() {
-    static int v = -1;
-    if (v < 0) {
-        const char *e = getenv("PSML_CONV_GW");
-        v = (e && e[0] == 'g') ? 0 : 1;
-    }
-    return v == 1;
-}
+// psml_options.conv_gw = 0 keeps the weight gradient on the generic im2col GEMM (tests)
+inline bool conv_gw_enabled() { return cur_opts().conv_gw != 0; }
 
 // The fast path applies to the untruncated weight gradient in Z_2^64 with N % 4 == 0 and
 // operands that fit shared memory; false -> the generic im2col GEMM.

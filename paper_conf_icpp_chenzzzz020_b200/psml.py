@@ -35,6 +35,44 @@ class Ring(ctypes.Structure):
     _fields_ = [("l", i32), ("frac_bits", i32)]
 
 
+class Options(ctypes.Structure):
+    """psml_options (include/psml.h): explicit per-context execution options."""
+    _fields_ = [(n, i32) for n in ("seg_backend", "pdl", "fused_open", "fused_step", "fused_dealer",
+                                    "deal_split", "deal_after", "gradw_branch", "simt_cluster",
+                                    "rows_kernel", "msb_chain", "conv_gw")]
+
+
+# Test-harness convenience of the BINDING (the library reads no environment): PSML_* variables
+# override the defaults of every context this process creates, so a subprocess test can select an
+# alternative implementation; the values map to explicit psml_options fields.
+_ENV_OPTIONS = {
+    "PSML_SEG": ("seg_backend", {"simt": 1, "tc": 2}),
+    "PSML_PDL": ("pdl", {"0": 0, "1": 1}),
+    "PSML_OPEN": ("fused_open", {"fused": 1, "mask": 0}),
+    "PSML_FUSE": ("fused_step", {"0": 0, "1": 1}),
+    "PSML_DEAL": ("fused_dealer", {"items": 0, "fused": 1}),
+    "PSML_DEAL_SPLIT": ("deal_split", {"0": 0, "1": 1}),
+    "PSML_DEAL_AFTER": ("deal_after", None),
+    "PSML_GRADW_BRANCH": ("gradw_branch", {"0": 0, "1": 1}),
+    "PSML_SIMT": ("simt_cluster", {"small": 0, "cluster": 1}),
+    "PSML_ROWS": ("rows_kernel", {"0": 0, "1": 1}),
+    "PSML_MSB_CHAIN": ("msb_chain", {"rounds": 1, "pair": 0}),
+    "PSML_CONV_GW": ("conv_gw", {"generic": 0, "image": 1}),
+}
+
+
+def default_options(**overrides):
+    o = Options()
+    _call("psml_options_default", ctypes.byref(o))
+    for var, (field, table) in _ENV_OPTIONS.items():
+        v = os.environ.get(var)
+        if v is not None:
+            setattr(o, field, int(v) if table is None else table.get(v, getattr(o, field)))
+    for k, v in overrides.items():
+        setattr(o, k, v)
+    return o
+
+
 class Trace(ctypes.Structure):
     _fields_ = [("E", vp * 2), ("E_open", vp), ("F", vp * 2), ("F_open", vp)]
 
@@ -63,6 +101,8 @@ _SIGS = {
     "psml_bench_mac_peak": (i32, [i32, vp]),
     "psml_ctx_create": (i32, [Ring, i32, vp]),
     "psml_ctx_destroy": (i32, [vp]),
+    "psml_options_default": (i32, [vp]),
+    "psml_ctx_set_options": (i32, [vp, vp]),
     "psml_prg_fill": (i32, [Ring, u64, u32, u64, u64, i64, vp, vp]),
     "psml_encode": (i32, [Ring, vp, i64, vp, vp]),
     "psml_decode": (i32, [Ring, vp, i64, vp, vp]),
@@ -268,8 +308,9 @@ def device_info():
 class Ctx:
     """psml_ctx: one per GPU and host thread.  backend: 0 auto, 1 CUDA-core, 2 tcgen05."""
 
-    def __init__(self, l=64, frac_bits=13, backend=0, party=None, xport=None, dp=None):
-        """party/xport/dp: a per-party context (psml_ctx_create_party) for psml_secure_matmul_party."""
+    def __init__(self, l=64, frac_bits=13, backend=0, party=None, xport=None, dp=None, options=None):
+        """party/xport/dp: a per-party context (psml_ctx_create_party) for psml_secure_matmul_party;
+        options: psml_options overrides (dict), on top of the defaults (default_options)."""
         self.ring = Ring(l, frac_bits)
         self.l = l
         self.party = party
@@ -281,6 +322,8 @@ class Ctx:
             _call("psml_ctx_create_party", self.ring, backend, party, xport.handle, dp.handle if dp else None,
                   ctypes.byref(h))
         self.handle = h
+        self.options = default_options(**(options or {}))
+        _call("psml_ctx_set_options", self.handle, ctypes.byref(self.options))
 
     def close(self):
         if self.handle:

@@ -33,8 +33,8 @@ def test_no_gpu_fails_loudly():
     with pytest.raises(psml.PsmlError) as e:
         psml.Ctx()
     assert e.value.status == 4  # PSML_ERR_UNSUPPORTED, never a CPU fallback
-    assert psml.msb_material_words(psml.Ring(64, 13), 10) == (6 * 6 + 2) * 10
-    assert psml.msb_material_words(psml.Ring(32, 13), 10) == (6 * 5 + 2) * 10
+    assert psml.msb_material_words(psml.Ring(64, 13), 10) == 11 * 10   # reduced prefix (R27)
+    assert psml.msb_material_words(psml.Ring(32, 13), 10) == 11 * 10
 
 
 def test_binding_rejects_wrong_buffers_before_the_abi():
