@@ -242,8 +242,19 @@ def make_transport(party, peer, group=None, kind="peer", capacity_bytes=64 << 20
     from . import psml
     if kind == "peer":
         xp, blob = psml.Transport.peer(party, capacity_bytes)
-        xp.connect(_swap_bytes(blob, party, peer, group))
-        return xp
+        ok = 1
+        try:
+            xp.connect(_swap_bytes(blob, party, peer, group))
+        except psml.PsmlError:   # e.g. no peer access between the two GPUs: both sides fall back
+            ok = 0
+        ok_peer = int.from_bytes(_swap_bytes(bytes([ok]), party, peer, group), "little")
+        if ok and ok_peer:
+            return xp
+        xp.close()
+        import sys
+        print("psml: peer-memory transport unavailable between the pair's GPUs; using NCCL send/recv",
+              file=sys.stderr)
+        kind = "nccl"
     if kind == "nccl":
         uid = psml.nccl_unique_id() if party == 0 else bytes(128)
         got = _swap_bytes(uid, party, peer, group)
