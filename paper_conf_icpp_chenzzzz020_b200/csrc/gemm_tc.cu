@@ -20,6 +20,9 @@
 // warp 2 = TMEM allocator; all four warps run the epilogue (warp w owns TMEM lanes 32w..32w+31).
 // Tile: 128 x BN (BN = 64 for l = 64: 8 shift accumulators x 64 columns = all 512 TMEM columns;
 // BN = 128 for l = 32: 4 x 128).  K block 32 bytes per stage, 4 (l=64) / 6 (l=32) stages.
+#ifndef PSML_TC_MINKB
+#define PSML_TC_MINKB 4   // fewest K blocks per split-K slice (512^3: 50 -> 44 us vs 8)
+#endif
 #include "engine.h"
 
 namespace psml {
@@ -600,7 +603,7 @@ static psml_status launch_gemm(TcParams<typename Cfg<l>::T> P, int64_t Mp, int64
     const int64_t tiles = (Mp / BM) * (Np / BN) * P.nparty;   // CTAs per split (pairs count 2)
     int splits = 1;
     if (tiles < sm_count)
-        splits = (int)std::min<int64_t>((sm_count + tiles - 1) / tiles, std::max(1, nkb / 8));
+        splits = (int)std::min<int64_t>((sm_count + tiles - 1) / tiles, std::max(1, nkb / PSML_TC_MINKB));
     splits = std::max(splits, (nkb + Cfg<l>::MAX_KB - 1) / Cfg<l>::MAX_KB);
     int kbs = (nkb + splits - 1) / splits;
     splits = (nkb + kbs - 1) / kbs;
