@@ -116,6 +116,9 @@ typedef struct {
     int32_t rows_kernel;   /* CNN tall-skinny conv products: 1 rows kernel, 0 small tile        */
     int32_t msb_chain;     /* MSB chain: 0 one lane-pair launch, 1 one kernel per round        */
     int32_t conv_gw;       /* CNN weight gradient: 1 per-image kernel, 0 generic im2col GEMM    */
+    int32_t split_fused;   /* split deployment over a peer transport: 1 each activation is ONE
+                              kernel with its 9 rounds' exchanges fused over peer memory, 0 one
+                              kernel + one exchange per round                                   */
 } psml_options;
 psml_status psml_options_default(psml_options *out);
 psml_status psml_ctx_set_options(psml_ctx ctx, const psml_options *opts);

@@ -291,7 +291,7 @@ psml_status psml_secure_matmul_party(psml_ctx ctx, const void *A_i, const void *
 }
 
 namespace psml {
-static const psml_options k_default_opts{0, 1, 0, 1, 1, 1, 1, 1, 1, 1, 0, 1};
+static const psml_options k_default_opts{0, 1, 0, 1, 1, 1, 1, 1, 1, 1, 0, 1, 1};
 static thread_local const psml_options *t_opts = nullptr;
 const psml_options &cur_opts() { return t_opts ? *t_opts : k_default_opts; }
 OptScope::OptScope(const psml_options *o) : prev(t_opts) { if (o) t_opts = o; }

@@ -8,6 +8,19 @@
 namespace psml {
 
 psml_status check_ring(psml_ring r);
+
+// Peer-memory window of a connected peer transport for FUSED compute + exchange kernels (split
+// deployment): this party's window (written by the peer), the peer's window (mapped), and the
+// flag words -- an epoch counter and a done counter per call, one release/acquire flag per CTA.
+constexpr int PW_MAX_CTAS = 64, PW_FLAG_STRIDE = 16, PW_EPOCH = 80, PW_DONE = 96, PW_FLAG_BASE = 128;
+constexpr int64_t PW_BYTES = (int64_t)8 << 20;
+struct PeerWindow {
+    uint8_t *my_win, *peer_win;
+    int64_t bytes;
+    uint64_t *my_flags, *peer_flags;
+};
+bool xport_peer_window(psml_xport x, PeerWindow *w);   // false: not a connected peer transport
+void xport_account(psml_xport x, int64_t exchanges, int64_t bytes);   // stats of fused exchanges
 // run the rest of an ABI call with the options of ctx / model (null: defaults)
 #define PSML_CTX_OPTS(c) ::psml::OptScope _psml_opts_((c) ? &reinterpret_cast<const ::psml::Ctx *>(c)->opts : nullptr)
 psml_status check_ptrs(std::initializer_list<const void *> ps);
@@ -16,7 +29,7 @@ int current_sm_count();
 struct Ctx {
     psml_ring ring{64, 13};
     int backend = 0;    // 0 auto, 1 CUDA-core, 2 tcgen05
-    psml_options opts{0, 1, 0, 1, 1, 1, 1, 1, 1, 1, 0, 1};   // = psml_options_default
+    psml_options opts{0, 1, 0, 1, 1, 1, 1, 1, 1, 1, 0, 1, 1};   // = psml_options_default
     int sm_count = 148;
     bool tc_ok = false;
     void *ws = nullptr;

@@ -20,6 +20,7 @@
 #include "dealer_fused.cuh"
 #include "fused.cuh"
 #include "fss.cuh"
+#include "split_fused.cuh"
 
 namespace psml {
 
@@ -1288,6 +1289,23 @@ static psml_status party_chain_fss(PartyRun &r, const T *x, const DealItem *mat,
 static psml_status party_chain(PartyRun &r, const T *x, const DealItem *mat, const DealItem *h, int what, T *y,
                                T *drelu, const T *Ysub, T *delta) {
     if (mat->kind == IT_FSS) return party_chain_fss(r, x, mat, h, what, y, drelu, Ysub, delta);
+    PeerWindow w;
+    if (mat->kind == IT_MSB && cur_opts().split_fused && xport_peer_window(r.x, &w)) {
+        // one kernel per party: the 9 rounds' exchanges fused over the peer window (split_fused.cuh)
+        ChainParty A{};
+        A.p = r.p; A.x = x; A.mat = mat->mat.p[r.p];
+        A.U = h->U.p[r.p]; A.V = h->V.p[r.p]; A.Z = h->Z.p[r.p];
+        A.y = y; A.drelu = drelu; A.Ysub = Ysub; A.delta = delta;
+        A.n = mat->n; A.what = what;
+        A.half = what == 2 ? (T)1 << (r.m->ctx->ring.frac_bits - 1) : 0;
+        A.w = w;
+        {
+            ProfScope prof(PROF_MSB, r.s, 0.0);
+            PSML_TRY(launch_chain_party(A, r.s));
+        }
+        xport_account(r.x, 9, 17 * 8 * mat->n);
+        return PSML_OK;
+    }
     psml_model_s *m = r.m;
     const int p = r.p, q = 1 - p;
     const int64_t n = mat->n;

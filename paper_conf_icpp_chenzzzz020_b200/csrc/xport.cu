@@ -22,10 +22,12 @@
 #include <string>
 #include <vector>
 
-#include "common.cuh"
+#include "engine.h"
 
-// flag words of a peer mailbox (each on its own 128-byte line)
-enum { XF_ARRIVED = 0, XF_CONSUMED = 16, XF_SEQ = 32, XF_CNT1 = 48, XF_CNT2 = 64, XF_WORDS = 80 };
+// flag words of a peer mailbox (each on its own 128-byte line); then the fused kernels' window
+// flags (psml::PeerWindow: an epoch counter, a done counter and one flag per CTA)
+enum { XF_ARRIVED = 0, XF_CONSUMED = 16, XF_SEQ = 32, XF_CNT1 = 48, XF_CNT2 = 64,
+       XF_WORDS = psml::PW_FLAG_BASE + psml::PW_MAX_CTAS * psml::PW_FLAG_STRIDE };
 
 struct psml_xport_s {
     int kind = 0;                 // 0 NCCL, 1 callback, 2 peer memory
@@ -248,7 +250,9 @@ psml_status psml_xport_peer_create(int32_t party, int64_t capacity_bytes, psml_x
     x->rank = party;
     x->device = dev;
     x->cap = cap;
-    if (cudaMalloc(&x->my_mb, 2 * cap) != cudaSuccess || cudaMalloc(&x->my_flags, XF_WORDS * sizeof(uint64_t)) != cudaSuccess) {
+    // two exchange slots + the fused kernels' window (PeerWindow), one allocation / one IPC handle
+    if (cudaMalloc(&x->my_mb, 2 * cap + PW_BYTES) != cudaSuccess ||
+        cudaMalloc(&x->my_flags, XF_WORDS * sizeof(uint64_t)) != cudaSuccess) {
         if (x->my_mb) cudaFree(x->my_mb);
         delete x;
         cudaGetLastError();
@@ -408,6 +412,24 @@ psml_status psml_dp_allreduce(psml_dp d, void *buf, int64_t n, int32_t l, psml_s
     if (r != ncclSuccess) return nccl_fail(r, "ncclAllReduce");
     return PSML_OK;
 }
+
+namespace psml {
+void xport_account(psml_xport x, int64_t exchanges, int64_t bytes) {
+    if (!x) return;
+    x->exchanges += exchanges;
+    x->bytes_sent += bytes;
+}
+
+bool xport_peer_window(psml_xport x, PeerWindow *w) {
+    if (!x || x->kind != 2 || !x->peer_mb || !w) return false;
+    w->my_win = x->my_mb + 2 * x->cap;
+    w->peer_win = x->peer_mb + 2 * x->cap;
+    w->bytes = PW_BYTES;
+    w->my_flags = x->my_flags;
+    w->peer_flags = x->peer_flags;
+    return true;
+}
+}  // namespace psml
 
 psml_status psml_xport_stats(psml_xport x, int64_t *bytes_sent, int64_t *exchanges) {
     if (!x) return fail(PSML_ERR_INVALID, "transport is null");

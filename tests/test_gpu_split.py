@@ -168,6 +168,9 @@ def _party_train(rank, port, outdir, kind, compare="a2b", mask_reuse=False):
     from paper_conf_icpp_chenzzzz020_b200.parallel import make_dp, make_transport
     from paper_conf_icpp_chenzzzz020_b200.train import PartyTrainer
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    if kind == "peer_rounds":           # one kernel + one exchange per round instead of the fused chain
+        os.environ["PSML_SPLIT_FUSED"] = "0"
+        kind = "peer"
     dist.init_process_group("gloo", rank=rank, world_size=2)
     torch.cuda.set_device(0)
     xp = make_transport(rank, 1 - rank, kind=kind)
@@ -206,11 +209,13 @@ def _check_against_oracle(tmp_path, tasks, compare="a2b", mask_reuse=False):
                         (task, s, layer, p)
 
 
-@pytest.mark.parametrize("kind", ["peer", "callback"])
+@pytest.mark.parametrize("kind", ["peer", "peer_rounds", "callback"])
 def test_split_training_matches_oracle(tmp_path, kind):
-    """Two party processes on the one test GPU.  kind=peer: every opening is the library's
-    peer-memory exchange kernel over CUDA-IPC-mapped mailboxes (device to device, no host hop);
-    kind=callback: host-staged gloo.  Each party's master shares equal the oracle's."""
+    """Two party processes on the one test GPU.  kind=peer: every Beaver opening is the library's
+    peer-memory exchange kernel over CUDA-IPC-mapped mailboxes and every activation ONE kernel with
+    its rounds' exchanges fused over the peer window (split_fused.cuh); peer_rounds: one kernel + one
+    exchange per activation round; callback: host-staged gloo.  Each party's master shares equal
+    the oracle's."""
     mp.spawn(_party_train, args=(_free_port(), str(tmp_path), kind), nprocs=2, join=True)
     _check_against_oracle(tmp_path, SPLIT_TASKS)
     st = [np.load(tmp_path / f"xstats_{p}.npy") for p in range(2)]
