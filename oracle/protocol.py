@@ -59,8 +59,9 @@ def dims_of(task):
 def share_batch(X, Y, step, pair=0):
     x = core.encode(X, L, F)
     y = core.encode(Y, L, F)
-    return (core.share(x, SHARE_SEED, call_id(pair, step, 0, OP_SHARE, 0)),
-            core.share(y, SHARE_SEED, call_id(pair, step, 0, OP_SHARE, 1)))
+    pf = _field(pair)   # strong scaling: each pair's client shares its own rows afresh
+    return (core.share(x, SHARE_SEED, call_id(pf, step, 0, OP_SHARE, 0)),
+            core.share(y, SHARE_SEED, call_id(pf, step, 0, OP_SHARE, 1)))
 
 
 def trunc_pair(x, d):
@@ -134,6 +135,61 @@ def _T(p):
     return np.ascontiguousarray(p[0].T), np.ascontiguousarray(p[1].T)
 
 
+class Strong:
+    """Pair k of P under strong scaling (R28): the P pairs train on ONE
+    global batch of P b rows, pair k on rows [k b, (k + 1) b).  Every op whose output rows are
+    batch rows -- forward and input-gradient products, ReLU / Eq. 9, Hadamard -- takes the
+    row-slices of the material a single pair would draw for the whole global batch (pair field 0;
+    the weight mask V is the global one, shared: every pair opens the same F = W - V of the same
+    replicated W).  Weight-gradient products contract over the batch and take independent
+    per-pair triplets (pair field k).  A mask is never reused on two different values."""
+
+    def __init__(self, k, P):
+        assert 0 <= k < P
+        self.k, self.P = k, P
+
+
+def _field(pair):
+    """Call-id pair field of a pair's own (per-pair) material."""
+    return pair.k if isinstance(pair, Strong) else pair
+
+
+def _slice_idx(pair, n, parts):
+    """Global element indices of pair k's n elements: `parts` row-ordered blocks of n / parts
+    (Eq. 9's [z + 1/2 ; z - 1/2]), block h of the global layout holding P n / parts elements."""
+    per = n // parts
+    return np.concatenate([h * pair.P * per + pair.k * per + np.arange(per) for h in range(parts)])
+
+
+def mat_triplet(pair, step, layer, op, M, K, N):
+    """Matrix triplet of the product (layer, op) with M output rows."""
+    if isinstance(pair, Strong) and op != OP_GRADW:
+        U0, U1, V0, V1, Z0, Z1 = core.triplet_gen(DEALER_SEED, call_id(0, step, layer, op, 0), pair.P * M, K, N, L)
+        r = slice(pair.k * M, (pair.k + 1) * M)
+        return U0[r], U1[r], V0, V1, Z0[r], Z1[r]
+    return core.triplet_gen(DEALER_SEED, call_id(_field(pair), step, layer, op, 0), M, K, N, L)
+
+
+def had_triplet(pair, step, layer, slot, n, parts=1):
+    if isinstance(pair, Strong):
+        t = core.hadamard_triplet_gen(DEALER_SEED, call_id(0, step, layer, OP_HADAMARD, slot), pair.P * n, L)
+        i = _slice_idx(pair, n, parts)
+        return tuple(a[i] for a in t)
+    return core.hadamard_triplet_gen(DEALER_SEED, call_id(pair, step, layer, OP_HADAMARD, slot), n, L)
+
+
+def cmp_material(pair, step, layer, op, n, compare, parts=1):
+    """Comparison material of n elements: A2B chain (R9, 11 planes of n words) or DCF keys (R22,
+    257 planes); plane-major, so a pair's slice is the same element range of every plane."""
+    gen = core.fss_dealer if compare == "fss" else core.msb_dealer
+    if isinstance(pair, Strong):
+        ng = pair.P * n
+        i = _slice_idx(pair, n, parts)
+        return tuple(np.ascontiguousarray(m.reshape(-1, ng)[:, i]).reshape(-1)
+                     for m in gen(DEALER_SEED, call_id(0, step, layer, op, 0), ng, L))
+    return gen(DEALER_SEED, call_id(pair, step, layer, op, 0), n, L)
+
+
 def reuse_triplets(pair, step, layer, B, din, dout):
     """SecureML forward/backward mask reuse (R26): the backward
     products of layer l re-use the masks of values already opened -- the activation A_l's forward
@@ -142,6 +198,7 @@ def reuse_triplets(pair, step, layer, B, din, dout):
     (gradW's right operand and gradin's left operand).  D_i = PRG("U0"/"U1") and Z_0 = PRG("Z0")
     under the gradin call id, Z_0 of gradW under the gradW call id; Z_1 = U V - Z_0 as usual.
     Returns (gradW triplet, gradin triplet) in core.triplet_gen's (U0, U1, V0, V1, Z0, Z1) order."""
+    assert not isinstance(pair, Strong), "mask reuse is not defined for the strong-scaling layout"
     Uf0, Uf1, Vf0, Vf1, _, _ = core.triplet_gen(DEALER_SEED, call_id(pair, step, layer, OP_FWD, 0), B, din, dout, L)
     cgi, cgw = call_id(pair, step, layer, OP_GRADIN, 0), call_id(pair, step, layer, OP_GRADW, 0)
     D0 = core.dealer_prg(L, DEALER_SEED, core.tag("U0"), cgi, B * dout).reshape(B, dout)
@@ -164,7 +221,7 @@ def matmul(A, B, pair, step, layer, op, trunc):
     """Beaver product of two shared matrices with the triplet of call id (pair,step,layer,op)."""
     M, K = A[0].shape
     N = B[0].shape[1]
-    trip = core.triplet_gen(DEALER_SEED, call_id(pair, step, layer, op, 0), M, K, N, L)
+    trip = mat_triplet(pair, step, layer, op, M, K, N)
     c = core.beaver_matmul(A, B, trip, trunc=0, l=L)   # Eq. 6/8, then truncation (R7)
     return checked_trunc(c, trunc) if trunc else c
 
@@ -173,13 +230,13 @@ def relu(z, pair, step, layer, compare="a2b"):
     """Secure ReLU: DReLU by the Kogge-Stone A2B chain (R9) or by the one-round FSS comparison
     (compare="fss", R22: material keyed by the same call id), then one Beaver Hadamard."""
     n = z[0].size
-    cid = call_id(pair, step, layer, OP_RELU_MSB, 0)
-    ht = core.hadamard_triplet_gen(DEALER_SEED, call_id(pair, step, layer, OP_HADAMARD, 0), n, L)
+    ht = had_triplet(pair, step, layer, 0, n)
+    mat = cmp_material(pair, step, layer, OP_RELU_MSB, n, compare)
     flat = (z[0].reshape(-1), z[1].reshape(-1))
     if compare == "fss":
-        (r0, r1), (d0, d1) = core.secure_relu_fss(flat, core.fss_dealer(DEALER_SEED, cid, n, L), ht, L)
+        (r0, r1), (d0, d1) = core.secure_relu_fss(flat, mat, ht, L)
     else:
-        (r0, r1), (d0, d1) = core.secure_relu(flat, core.msb_dealer(DEALER_SEED, cid, n, L), ht, L)
+        (r0, r1), (d0, d1) = core.secure_relu(flat, mat, ht, L)
     if DIAG["on"]:   # DReLU = 1 - MSB(x) must equal [x >= 0] on the plaintext
         x = _signed(z[0].reshape(-1) + z[1].reshape(-1))
         dr = np.asarray(d0 + d1, dtype=np.uint64)
@@ -191,15 +248,15 @@ def relu(z, pair, step, layer, compare="a2b"):
 
 def eq9(z, pair, step, layer, compare="a2b"):
     n = z[0].size
-    cid = call_id(pair, step, layer, OP_EQ9_MSB, 0)
-    ht = core.hadamard_triplet_gen(DEALER_SEED, call_id(pair, step, layer, OP_HADAMARD, 2), 2 * n, L)
+    ht = had_triplet(pair, step, layer, 2, 2 * n, parts=2)
+    mat = cmp_material(pair, step, layer, OP_EQ9_MSB, 2 * n, compare, parts=2)
     if compare == "fss":   # Eq. 9 = ReLU(x + 1/2) - ReLU(x - 1/2) with the FSS ReLU (R22)
         x = core.eq9_inputs(z, L, F)
-        (r0, r1), _ = core.secure_relu_fss(x, core.fss_dealer(DEALER_SEED, cid, 2 * n, L), ht, L)
+        (r0, r1), _ = core.secure_relu_fss(x, mat, ht, L)
         shape = np.shape(z[0])
         y = (((r0[:n] - r0[n:]) & MASK).reshape(shape), ((r1[:n] - r1[n:]) & MASK).reshape(shape))
     else:
-        y = core.secure_eq9(z, core.msb_dealer(DEALER_SEED, cid, 2 * n, L), ht, L, F)
+        y = core.secure_eq9(z, mat, ht, L, F)
     if DIAG["on"]:   # Eq. 9 on the grid: clamp(x + 2^(F-1), 0, 2^F) exactly (R8)
         x = _signed(z[0] + z[1])
         want = np.clip(x + (1 << (F - 1)), 0, 1 << F)
@@ -210,7 +267,7 @@ def eq9(z, pair, step, layer, compare="a2b"):
 
 def hadamard(a, b, pair, step, layer, slot):
     n = a[0].size
-    ht = core.hadamard_triplet_gen(DEALER_SEED, call_id(pair, step, layer, OP_HADAMARD, slot), n, L)
+    ht = had_triplet(pair, step, layer, slot, n)
     c0, c1 = core.beaver_hadamard((a[0].reshape(-1), a[1].reshape(-1)),
                                   (b[0].reshape(-1), b[1].reshape(-1)), ht, L)
     return c0.reshape(a[0].shape), c1.reshape(a[0].shape)
@@ -220,6 +277,7 @@ def hadamard(a, b, pair, step, layer, slot):
 def conv_triplet(pair, step, op, B, transpose):
     """U over the raw input (B x C*H*W), V, Z = im2col(U).V (op 0) or im2col(U)^T.V (op 1)."""
     g = CNN_GEOM
+    assert not isinstance(pair, Strong), "the strong-scaling layout is not defined for the CNN"
     cid = call_id(pair, step, 0, op, 0)
     nin = B * g["C"] * g["H"] * g["W"]
     rows = B * (g["H"] - g["k"] + 1) * (g["W"] - g["k"] + 1)
@@ -259,13 +317,13 @@ def comparison_lt0(t, pair, step, layer, compare="a2b"):
     """Arithmetic shares of [t < 0] (signed) = MSB(t): the A2B chain's MSB (R9), or 1 - DReLU from
     the FSS comparison (R22).  Material keyed like ReLU's (op 3)."""
     n = t[0].size
-    cid = call_id(pair, step, layer, OP_RELU_MSB, 0)
+    mat = cmp_material(pair, step, layer, OP_RELU_MSB, n, compare)
     flat = (t[0].reshape(-1), t[1].reshape(-1))
     if compare == "fss":
-        d0, d1 = core.fss_drelu(flat, core.fss_dealer(DEALER_SEED, cid, n, L), L)
+        d0, d1 = core.fss_drelu(flat, mat, L)
         out = ((np.uint64(1) - d0) & MASK, (np.uint64(0) - d1) & MASK)
     else:
-        out = core.secure_msb(flat, core.msb_dealer(DEALER_SEED, cid, n, L), L)
+        out = core.secure_msb(flat, mat, L)
     if DIAG["on"]:
         x = _signed(flat[0] + flat[1])
         DIAG["msb_checked"] += int(x.size)
@@ -412,6 +470,25 @@ def apply_update(model, grads, n_pairs=1):
             gt = (gt[0] + trunc_pair(model.Wm[layer], WD_SHIFT)[0], gt[1] + trunc_pair(model.Wm[layer], WD_SHIFT)[1])
         model.Wm[layer] = sub_pair(model.Wm[layer], gt)
         model.W[layer] = checked_trunc(model.Wm[layer], MASTER - model.fw[layer])
+
+
+def strong_forward_backward(model, Xs, Ys, step, P):
+    """Strong scaling over P pairs (R28), every pair simulated: Xs / Ys are
+    the global batch's shares; pair k runs forward / backward on rows [k b, (k + 1) b) with the
+    Strong(k, P) material, and each party's weight-gradient shares are summed over the P pairs
+    (the per-party all-reduce; ring addition, exact).  The sum is the global batch's gradient, so
+    the update takes no extra shift (apply_update(..., n_pairs=1)).  Returns (summed gradient
+    shares, per-pair prediction shares stacked in row order)."""
+    B = Xs[0].shape[0]
+    assert B % P == 0
+    b = B // P
+    total, yh = None, []
+    for k in range(P):
+        r = slice(k * b, (k + 1) * b)
+        g, y = forward_backward(model, (Xs[0][r], Xs[1][r]), (Ys[0][r], Ys[1][r]), step, Strong(k, P))
+        total = g if total is None else [(t[0] + u[0], t[1] + u[1]) for t, u in zip(total, g)]
+        yh.append(y)
+    return total, (np.concatenate([y[0] for y in yh]), np.concatenate([y[1] for y in yh]))
 
 
 def train_step(model, X, Y, step, pair=0):
