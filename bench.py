@@ -11,7 +11,8 @@ truncation, secure ReLU / Eq. 9, backprop, master-weight update) -- DESIGN.md "M
 N > 1 (torchrun): the split deployment -- party 0 on GPU k, party 1 on GPU k + N/2, N/2 pairs
 each on its own 128 rows (weak scaling), every opening one peer-memory exchange over NVLink,
 per-party NCCL all-reduce of the gradient shares, one CUDA graph per party step
-(`--deployment coresident`: one co-resident pair per GPU instead).
+(`--deployment coresident`: one co-resident pair per GPU instead; `--scaling strong`: ONE global
+batch of 128 rows split over the pairs with the row-sliced dealer layout).
 Timing: W untimed warm-up steps, then K steps each bracketed by CUDA events on the launching
 stream with a 256 MiB L2 flush between steps (outside the events); barrier + synchronize around
 the timed region; the max over ranks.  `--impl reference` times the CPU oracle instead.
@@ -65,6 +66,10 @@ def parse():
                          "opening round one peer-memory exchange over NVLink (SURVEY 8(e)); "
                          "coresident: both parties of a pair on one GPU; auto (default): split for "
                          "N >= 2, coresident for N = 1")
+    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
+                    help="N > 1: weak = 128 rows per pair (global batch 128 x pairs); strong = ONE global "
+                         "batch of 128 rows split over the pairs with the row-sliced dealer layout "
+                         "(SURVEY C16, DESIGN.md R28)")
     a = ap.parse_args()
     global TASK, WORKLOAD
     TASK, WORKLOAD = a.task, WORKLOADS[a.task]
@@ -160,6 +165,23 @@ def dist_setup(args):
     return world, rank, local
 
 
+def pair_batch(args, s, pair, pairs, u8=False):
+    """Minibatch rows of pair `pair` of `pairs` for step s: its own 128 rows (weak scaling) or its
+    slice of ONE global batch of 128 rows (strong scaling, parallel.strong_rows)."""
+    import synth
+    gen = synth.batch_u8 if u8 else synth.batch
+    if args.scaling == "strong" and pairs > 1:
+        from paper_conf_icpp_chenzzzz020_b200.parallel import strong_rows
+        X, Y = gen(TASK, s, BATCH)
+        r = strong_rows(pair, pairs, BATCH)
+        return X[r], Y[r]
+    return gen(TASK, s, BATCH, pair=pair, n_pairs=pairs)
+
+
+def per_pair_rows(args, pairs):
+    return BATCH // pairs if (args.scaling == "strong" and pairs > 1) else BATCH
+
+
 def max_over_ranks(x, world):
     if world == 1:
         return x
@@ -177,7 +199,7 @@ def bench_ours(args):
 
     import synth
     from paper_conf_icpp_chenzzzz020_b200 import build, psml
-    from paper_conf_icpp_chenzzzz020_b200.parallel import dp_update_shift, ring_allreduce_
+    from paper_conf_icpp_chenzzzz020_b200.parallel import ring_allreduce_
     from paper_conf_icpp_chenzzzz020_b200.train import SecureTrainer
 
     build.build()
@@ -185,19 +207,22 @@ def bench_ours(args):
     dev = torch.device("cuda", local)
     K, W = args.steps, args.warmup
     whole = ClockSampler(local).__enter__()   # clocks over the whole GPU-active bench
-    tr = SecureTrainer(TASK, synth.init_weights(TASK), batch=BATCH, pair_id=rank)
+    strong = args.scaling == "strong" and world > 1
+    rows = per_pair_rows(args, world)
+    tr = SecureTrainer(TASK, synth.init_weights(TASK), batch=rows, pair_id=rank, strong_pairs=world if strong else 0)
     # plaintext minibatches resident in HBM (and pinned host copies for the e2e leg)
     nb = K + W
     Xs, Ys = [], []
     for s in range(nb):
-        X, Y = synth.batch(TASK, s, BATCH, pair=rank, n_pairs=world)
-        Xs.append(torch.from_numpy(X).to(dev))
-        Ys.append(torch.from_numpy(Y).to(dev))
+        X, Y = pair_batch(args, s, rank, world)
+        Xs.append(torch.from_numpy(np.ascontiguousarray(X)).to(dev))
+        Ys.append(torch.from_numpy(np.ascontiguousarray(Y)).to(dev))
     # e2e leg: the client's own form of the same batches -- 8-bit pixels and (one-hot tasks)
     # class indices -- in pinned host memory; they share bit-identically to the float64 batches
     Xh, Yh = [], []
     for s in range(nb):
-        q, y = synth.batch_u8(TASK, s, BATCH, pair=rank, n_pairs=world)
+        q, y = pair_batch(args, s, rank, world, u8=True)
+        q = np.ascontiguousarray(q)
         Xh.append(torch.from_numpy(q).pin_memory())
         Yh.append(torch.from_numpy(np.ascontiguousarray(y)).pin_memory())
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
@@ -209,7 +234,7 @@ def bench_ours(args):
         tr.graph_step(X, Y, s)
         if world > 1:
             ring_allreduce_(tr.grad_tensor())
-            tr.model.apply_update(extra_shift=dp_update_shift(world))
+            tr.model.apply_update(extra_shift=tr.update_shift(world))
 
     def one_step(s, X, Y, online_only=False, shares=None):
         if online_only:
@@ -287,7 +312,7 @@ def bench_ours(args):
 
     # e2e through the public API with host buffers: H2D plaintext batch, full step, D2H yhat
     h2d = Xh[0].numel() * Xh[0].element_size() + Yh[0].numel() * Yh[0].element_size()
-    out_host = torch.empty((2, BATCH, Ys[0].shape[1]), dtype=torch.uint64).pin_memory()
+    out_host = torch.empty((2, rows, Ys[0].shape[1]), dtype=torch.uint64).pin_memory()
     d2h = out_host.numel() * 8
 
     def e2e_step(s):
@@ -313,14 +338,14 @@ def bench_ours(args):
         tr.infer_shares(Xsh, s)
     t_inf = max_over_ranks(timed(infer_step, K, 10 * (W + K)), world)
 
-    samples = BATCH * K * world
+    samples = rows * K * world
     result = {
         "metric": METRIC, "value": samples / t_dev, "unit": "samples/s", "n_gpus": world,
         "steps": K, "warmup": W, "ms_per_step": 1e3 * t_dev / K, "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": "u64",
+        "scaling": "strong" if strong else "weak", "vs_baseline": None, "dtype": "u64",
         "data": ("synthetic (CIFAR-shaped 3x32x32 8-bit pixels; teacher-CNN labels)" if TASK == "cnn" else
                  "synthetic (MNIST-shaped 8-bit pixels, 81% zeros; teacher labels)"),
-        "config": arm_config(world),
+        "config": arm_config(world, args.scaling),
         "online_samples_per_s": samples / t_on,
         "online_graph_samples_per_s": (samples / t_on_graph) if t_on_graph else None,
         "eager_samples_per_s": samples / t_eager,
@@ -405,16 +430,18 @@ def bench_split(args):
     cap = (96 << 20) if TASK == "cnn" else (8 << 20)
     xp = make_transport(party, peer, kind=os.environ.get("PSML_XPORT", "peer"), capacity_bytes=cap)
     dp = make_dp(list(range(party * half, (party + 1) * half)), rank, groups[party])
-    tr = PartyTrainer(TASK, synth.init_weights(TASK), party, xp, batch=BATCH, pair_id=pair, dp=dp,
-                      mask_reuse=args.mask_reuse, compare=args.compare)
+    strong = args.scaling == "strong" and half > 1
+    rows = per_pair_rows(args, half)
+    tr = PartyTrainer(TASK, synth.init_weights(TASK), party, xp, batch=rows, pair_id=pair, dp=dp,
+                      mask_reuse=args.mask_reuse, compare=args.compare, strong_pairs=half if strong else 0)
     nb = min(K + W, 64)
     Xs, Ys, Xh, Yh = [], [], [], []
     for s in range(nb):
-        X, Y = synth.batch(TASK, s, BATCH, pair=pair, n_pairs=half)
-        Xs.append(torch.from_numpy(X).to(dev))
-        Ys.append(torch.from_numpy(Y).to(dev))
-        q, y = synth.batch_u8(TASK, s, BATCH, pair=pair, n_pairs=half)
-        Xh.append(torch.from_numpy(q).pin_memory())
+        X, Y = pair_batch(args, s, pair, half)
+        Xs.append(torch.from_numpy(np.ascontiguousarray(X)).to(dev))
+        Ys.append(torch.from_numpy(np.ascontiguousarray(Y)).to(dev))
+        q, y = pair_batch(args, s, pair, half, u8=True)
+        Xh.append(torch.from_numpy(np.ascontiguousarray(q)).pin_memory())
         Yh.append(torch.from_numpy(np.ascontiguousarray(y)).pin_memory())
     stream = torch.cuda.current_stream()
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
@@ -451,7 +478,7 @@ def bench_split(args):
     with ClockSampler(local) as clk:
         t_dev = timed(step, K, W + 1)
     launches = psml.kernel_launch_count() - l0
-    out_host = torch.empty(BATCH * Ys[0].shape[1], dtype=torch.uint64).pin_memory()
+    out_host = torch.empty(rows * Ys[0].shape[1], dtype=torch.uint64).pin_memory()
     from paper_conf_icpp_chenzzzz020_b200.train import _wrap_device_ptr
 
     def e2e(s):
@@ -461,14 +488,14 @@ def bench_split(args):
         ptrs = tr.model.output()
         out_host.copy_(_wrap_device_ptr(ptrs[party], ptrs[2], "<u8"), non_blocking=True)
     t_e2e = timed(e2e, K, W + K + 1)
-    samples = BATCH * K * half
+    samples = rows * K * half
     return {
         "metric": METRIC, "value": samples / t_dev, "unit": "samples/s", "n_gpus": world,
         "steps": K, "warmup": W, "ms_per_step": 1e3 * t_dev / K, "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": "u64",
+        "scaling": "strong" if strong else "weak", "vs_baseline": None, "dtype": "u64",
         "data": "synthetic (MNIST-shaped 8-bit pixels, 81% zeros; teacher labels)",
         "config": {"workload": WORKLOAD, "deployment": "split (party 0 on GPU k, party 1 on GPU k + N/2)",
-                   "global_batch": BATCH * half, "per_pair_batch": BATCH, "pairs": half,
+                   "global_batch": rows * half, "per_pair_batch": rows, "pairs": half,
                    "ring": "Z_2^64, 13 fractional bits", "parallelism": f"{half} pairs x 2 parties",
                    "transport": xp_kind(), "mask_reuse": bool(args.mask_reuse), "compare": args.compare,
                    "l2": "256 MiB flush between timed steps (outside the events)",
@@ -957,9 +984,11 @@ def secondary_figures(K=50):
     return out
 
 
-def arm_config(world):
+def arm_config(world, scaling="weak"):
     """The `config` of both arms' JSON lines."""
-    return {"workload": WORKLOAD, "global_batch": BATCH * world, "per_pair_batch": BATCH,
+    strong = scaling == "strong" and world > 1
+    return {"workload": WORKLOAD, "global_batch": BATCH if strong else BATCH * world,
+            "per_pair_batch": BATCH // world if strong else BATCH,
             "ring": "Z_2^64, 13 fractional bits", "parallelism": f"dp{world} (pairs)",
             "l2": "256 MiB flush between timed steps (outside the events)",
             "step": "client encode+share, dealer (offline), online secure step"}
@@ -983,10 +1012,11 @@ def bench_reference(args, budget_s=150.0):
     return {
         "impl": "reference", "metric": METRIC, "value": v, "unit": "samples/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t / n,
-        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
+        "higher_is_better": True, "scaling": "strong" if (args.scaling == "strong" and world > 1) else "weak",
+        "vs_baseline": None, "dtype": "u64",
         "data": ("synthetic (CIFAR-shaped 3x32x32 8-bit pixels; teacher-CNN labels)" if TASK == "cnn" else
                  "synthetic (MNIST-shaped 8-bit pixels, 81% zeros; teacher labels)"),
-        "config": arm_config(world),
+        "config": arm_config(world, args.scaling),
         "cpu_baseline": {"value": v, "unit": "samples/s", "cores": cores, "kind": "oracle", "cpu_model": cpu_model(),
                          "sample": f"{n} of the {args.steps} requested steps: full oracle secure training "
                                    f"steps of batch {BATCH} (both parties simulated) on the host"},

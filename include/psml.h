@@ -346,6 +346,19 @@ typedef struct {
                                  that party's seed s_i = psml_dealer_party_seed(dealer seed, i));
                                  the words it cannot derive come in the dealer's bundle
                                  (psml_model_deal_bundle / psml_model_deal_party)              */
+    int32_t strong_pairs;     /* SURVEY C16 / DESIGN.md R28 strong scaling. 0 or 1: this pair's
+                                 material is its own (pair field = pair_id; weak scaling).
+                                 P >= 2: P pairs train on ONE global batch of P * batch rows, this
+                                 pair (pair_id < P) on rows [pair_id * batch, (pair_id + 1) * batch):
+                                 the forward / input-gradient products, ReLU / Eq. 9 and Hadamard
+                                 material is the row-slice of what a single pair would be dealt
+                                 for the global batch (pair field 0; the weight masks V global and
+                                 shared), the weight-gradient triplets are this pair's own (pair
+                                 field pair_id).  The per-party sum of the P pairs' gradient shares
+                                 is the global-batch gradient: update with extra_shift = 0.
+                                 Requires batch % 8 == 0 (ChaCha20 block-aligned slices), the
+                                 fused dealer (psml_options.fused_dealer), kinds LINREG, LOGREG,
+                                 MLP, SVM, RNN and mask_reuse = 0.                               */
 } psml_model_desc;
 
 psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_model *out);

@@ -23,6 +23,8 @@ struct PrgJob {
     uint32_t tag[5];
     uint64_t cid;         // call id with step field 0
     int64_t n;            // elements
+    int64_t boff;         // ChaCha20 block offset of element 0 in every stream of the job (the
+                          // strong-scaling row-slice of a global stream, R28)
     int64_t blk_begin;    // first global block of this job
     uint64_t *out[6];
 };
@@ -88,19 +90,20 @@ __global__ void __launch_bounds__(128, PSML_DEAL_MINB) deal_prg_kernel(const Prg
         }
         const PrgJob &J = jobs[lo];
         const int64_t b = g - J.blk_begin, e0 = b * 8, n = J.n;
+        const uint32_t ctr = (uint32_t)(b + J.boff);   // stream block of local block b
         const uint64_t cid = cid_with_step(J.cid, step);
         const int kind = J.kind;
         uint64_t v[8], x[8], y[8];
-        deal_block(dkey(S, J.tag[0], cid), (uint32_t)b, v);
+        deal_block(dkey(S, J.tag[0], cid), ctr, v);
         if (kind == PJ_DABIT) {
 #pragma unroll
             for (int j = 0; j < 8; ++j) { x[j] = v[j] & 1; }
             deal_store8(J.out[0], e0, n, x);
-            deal_block(dkey(S, J.tag[1], cid), (uint32_t)b, v);
+            deal_block(dkey(S, J.tag[1], cid), ctr, v);
 #pragma unroll
             for (int j = 0; j < 8; ++j) { v[j] &= 1; x[j] ^= v[j]; }
             deal_store8(J.out[1], e0, n, v);
-            deal_block(dkey(S, J.tag[2], cid), (uint32_t)b, v);   // r^A_0
+            deal_block(dkey(S, J.tag[2], cid), ctr, v);   // r^A_0
             deal_store8(J.out[2], e0, n, v);
 #pragma unroll
             for (int j = 0; j < 8; ++j) x[j] -= v[j];                    // r^A_1 = (r0 ^ r1) - r^A_0
@@ -112,19 +115,19 @@ __global__ void __launch_bounds__(128, PSML_DEAL_MINB) deal_prg_kernel(const Prg
 #pragma unroll
             for (int j = 0; j < 8; ++j) { v[j] &= mk; x[j] = v[j]; }
             deal_store8(J.out[0], e0, n, v);
-            deal_block(dkey(S, J.tag[1], cid), (uint32_t)b, v);
+            deal_block(dkey(S, J.tag[1], cid), ctr, v);
 #pragma unroll
             for (int j = 0; j < 8; ++j) { v[j] &= mk; x[j] ^= v[j]; }
             deal_store8(J.out[1], e0, n, v);
-            deal_block(dkey(S, J.tag[2], cid), (uint32_t)b, y);
+            deal_block(dkey(S, J.tag[2], cid), ctr, y);
 #pragma unroll
             for (int j = 0; j < 8; ++j) y[j] &= mk;
             deal_store8(J.out[2], e0, n, y);
-            deal_block(dkey(S, J.tag[3], cid), (uint32_t)b, v);
+            deal_block(dkey(S, J.tag[3], cid), ctr, v);
 #pragma unroll
             for (int j = 0; j < 8; ++j) { v[j] &= mk; x[j] &= y[j] ^ v[j]; }
             deal_store8(J.out[3], e0, n, v);
-            deal_block(dkey(S, J.tag[4], cid), (uint32_t)b, v);
+            deal_block(dkey(S, J.tag[4], cid), ctr, v);
 #pragma unroll
             for (int j = 0; j < 8; ++j) { v[j] &= mk; x[j] ^= v[j]; }
             deal_store8(J.out[4], e0, n, v);
@@ -135,10 +138,10 @@ __global__ void __launch_bounds__(128, PSML_DEAL_MINB) deal_prg_kernel(const Prg
         if (kind == PJ_SINGLE) continue;
 #pragma unroll
         for (int j = 0; j < 8; ++j) x[j] = v[j];
-        deal_block(dkey(S, J.tag[1], cid), (uint32_t)b, v);
+        deal_block(dkey(S, J.tag[1], cid), ctr, v);
         deal_store8(J.out[1], e0, n, v);
         if (kind == PJ_PAIR) continue;
-        deal_tail<true>(J, S, cid, (uint32_t)b, e0, n, x, v);   // PJ_HAD
+        deal_tail<true>(J, S, cid, ctr, e0, n, x, v);   // PJ_HAD
     }
 }
 

@@ -59,14 +59,18 @@ __device__ __forceinline__ uint64_t neg_if(int t, uint64_t v) { return t ? (uint
 
 // Dealer (offline): Gen of Fig. 1 for every element; both parties' material.
 static __global__ void __launch_bounds__(128) fss_dealer_kernel(PrgKey kr, PrgKey kr0, PrgKey ks0, PrgKey kk0, PrgKey kk1,
-                                                         int64_t n, uint64_t *__restrict__ mat0,
+                                                         int64_t n, int64_t e_lo, int64_t e_hi, int64_t eoff,
+                                                         uint64_t *__restrict__ mat0,
                                                          uint64_t *__restrict__ mat1) {
+    // elements [e_lo, e_hi) of an n-element material (plane pitch n); element e draws stream
+    // element es = e + eoff (eoff != 0: a strong-scaling row-slice of a global stream, R28)
     kr = live_key(kr); kr0 = live_key(kr0); ks0 = live_key(ks0); kk0 = live_key(kk0); kk1 = live_key(kk1);
-    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x) {
-        const uint64_t r = prg_elem<uint64_t>(kr, e), r0 = prg_elem<uint64_t>(kr0, e), sa0 = prg_elem<uint64_t>(ks0, e);
+    for (int64_t e = e_lo + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < e_hi; e += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t es = e + eoff;
+        const uint64_t r = prg_elem<uint64_t>(kr, es), r0 = prg_elem<uint64_t>(kr0, es), sa0 = prg_elem<uint64_t>(ks0, es);
         S128 s[2];
-        s[0].lo = prg_elem<uint64_t>(kk0, 2 * e); s[0].hi = prg_elem<uint64_t>(kk0, 2 * e + 1);
-        s[1].lo = prg_elem<uint64_t>(kk1, 2 * e); s[1].hi = prg_elem<uint64_t>(kk1, 2 * e + 1);
+        s[0].lo = prg_elem<uint64_t>(kk0, 2 * es); s[0].hi = prg_elem<uint64_t>(kk0, 2 * es + 1);
+        s[1].lo = prg_elem<uint64_t>(kk1, 2 * es); s[1].hi = prg_elem<uint64_t>(kk1, 2 * es + 1);
         const uint64_t sbit = r >> 63, alpha = r & (((uint64_t)1 << FSS_BITS) - 1);
         const uint64_t beta = (uint64_t)1 - 2 * sbit;
         mat0[e] = r0; mat1[e] = r - r0;
@@ -185,12 +189,15 @@ static __global__ void __launch_bounds__(256) eq9_combine_kernel(CPair<uint64_t>
 }
 
 // Dealer launch with keys whose step field may live in device memory (CUDA graphs).
+// elements [e_lo, e_hi) (e_hi < 0: n) of the n-element material, stream elements e + eoff
 static inline psml_status fss_dealer_launch(const DealSeeds &S, uint64_t cid, int64_t n, uint64_t *m0, uint64_t *m1,
-                                            cudaStream_t s, const uint32_t *step = nullptr) {
-    if (n <= 0) return PSML_OK;
-    fss_dealer_kernel<<<grid_for(n, 128, 148 * 16), 128, 0, s>>>(
+                                            cudaStream_t s, const uint32_t *step = nullptr, int64_t e_lo = 0,
+                                            int64_t e_hi = -1, int64_t eoff = 0) {
+    if (e_hi < 0) e_hi = n;
+    if (e_hi <= e_lo) return PSML_OK;
+    fss_dealer_kernel<<<grid_for(e_hi - e_lo, 128, 148 * 16), 128, 0, s>>>(
         dkey(S, TAG_FR, cid, step), dkey(S, TAG_F0, cid, step), dkey(S, TAG_FS, cid, step),
-        dkey(S, TAG_K0, cid, step), dkey(S, TAG_K1, cid, step), n, m0, m1);
+        dkey(S, TAG_K0, cid, step), dkey(S, TAG_K1, cid, step), n, e_lo, e_hi, eoff, m0, m1);
     PSML_LAUNCH_CHECK();
     return PSML_OK;
 }

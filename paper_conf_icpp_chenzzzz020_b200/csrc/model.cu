@@ -192,6 +192,25 @@ static void add_msb(psml_model_s *m, int layer, int op, int64_t n, bool fwd) {
     m->items[0].push_back(it);
 }
 
+// Strong-scaling view of a dealer item (R28): with strong_pairs = P > 1
+// every item whose output rows are batch rows is the row-slice of the material a single pair
+// would be dealt for the global batch (pair field 0, stream elements offset by the slice start);
+// the weight-gradient triplets (contractions over the batch) stay this pair's own.
+static bool strong_rows(const psml_model_s *m, const DealItem &it) {
+    return m->d.strong_pairs > 1 && !(it.kind == IT_MATRIX && it.op == OP_GRADW);
+}
+static uint32_t item_pair(const psml_model_s *m, const DealItem &it) { return strong_rows(m, it) ? 0u : m->d.pair_id; }
+// row-ordered parts of an elementwise item: Eq. 9's [z + 1/2 ; z - 1/2] material is 2 parts, so a
+// pair's slice is one range in each half of the global layout
+static int item_parts(const DealItem &it) {
+    const bool eq9 = ((it.kind == IT_MSB || it.kind == IT_FSS) && it.op == OP_EQ9_MSB) || (it.kind == IT_HAD && it.slot == 2);
+    return eq9 ? 2 : 1;
+}
+// stream element of local element h * per of part h (per = n / parts elements per part)
+static int64_t strong_elem0(const psml_model_s *m, int64_t per, int h) {
+    return ((int64_t)h * m->d.strong_pairs + m->d.pair_id) * per;
+}
+
 static bool is_eq9_out(const psml_model_s *m) { return m->d.kind != PSML_LINREG && m->d.kind != PSML_SVM; }
 // forward-weight fractional bits of layer l (R21)
 static int fw(const psml_model_s *m, int l) {
@@ -426,7 +445,7 @@ static psml_status deal_reuse_item(psml_model_s *m, DealItem &it, uint32_t step,
 
 static psml_status deal_item(psml_model_s *m, DealItem &it, uint32_t step, cudaStream_t s) {
     const uint64_t seed = m->d.dealer_seed;
-    const uint64_t cid = call_id(m->d.pair_id, step, it.layer, it.op, it.slot);
+    const uint64_t cid = call_id(item_pair(m, it), step, it.layer, it.op, it.slot);
     if (m->d.mask_reuse && it.kind == IT_MATRIX && (it.op == OP_GRADW || it.op == OP_GRADIN))
         return deal_reuse_item(m, it, step, s);
     switch (it.kind) {
@@ -447,7 +466,13 @@ static psml_status deal_item(psml_model_s *m, DealItem &it, uint32_t step, cudaS
     }
     case IT_FSS: {
         ProfScope prof(PROF_DEALER, s, 2.0 * FSS_BITS * (double)it.n);
-        return fss_dealer_launch(m->seeds, cid, it.n, it.mat.p[0], it.mat.p[1], s, m->step_dev);
+        if (!strong_rows(m, it)) return fss_dealer_launch(m->seeds, cid, it.n, it.mat.p[0], it.mat.p[1], s, m->step_dev);
+        const int parts = item_parts(it);
+        const int64_t per = it.n / parts;
+        for (int h = 0; h < parts; ++h)   // local [h per, (h + 1) per) <- global part h, this pair's rows
+            PSML_TRY(fss_dealer_launch(m->seeds, cid, it.n, it.mat.p[0], it.mat.p[1], s, m->step_dev, h * per,
+                                       (h + 1) * per, strong_elem0(m, per, h) - h * per));
+        return PSML_OK;
     }
     }
     return PSML_OK;
@@ -465,8 +490,9 @@ static psml_status build_plan(psml_model_s *m, int pool, bool infer_only) {
     const int gBK = P.gemm_big ? ClDealer::BK : ClDefault::BK;
     std::vector<PrgJob> pjm, pjr;   // matrix-triplet streams, then the rest
     std::vector<ClJob<DealerOps<T>>> gj;
+    // one job: n elements of every stream in `tags`, stream element e0 = boff * 8 first
     auto job = [&](int kind, std::initializer_list<uint32_t> tags, uint64_t cid, int64_t n,
-                   std::initializer_list<T *> outs) {
+                   std::initializer_list<T *> outs, int64_t boff) {
         if (n <= 0) return;
         PrgJob j{};
         j.kind = kind;
@@ -475,7 +501,7 @@ static psml_status build_plan(psml_model_s *m, int pool, bool infer_only) {
         for (uint32_t t : tags) j.tag[i++] = t;
         i = 0;
         for (T *o : outs) j.out[i++] = o;
-        j.cid = cid; j.n = n;
+        j.cid = cid; j.n = n; j.boff = boff;
         P.chacha_blocks += (double)((n + 7) / 8) * (double)tags.size();
         (kind == PJ_PAIR || kind == PJ_SINGLE ? pjm : pjr).push_back(j);
     };
@@ -483,14 +509,18 @@ static psml_status build_plan(psml_model_s *m, int pool, bool infer_only) {
     for (size_t k = 0; k < items.size(); ++k) {
         DealItem &it = items[k];
         if (infer_only && !it.fwd) continue;
-        const uint64_t cid = call_id(m->d.pair_id, 0, it.layer, it.op, it.slot);
+        const uint64_t cid = call_id(item_pair(m, it), 0, it.layer, it.op, it.slot);
+        // strong scaling (R28): this pair's rows of the global streams; U and Z row-sliced, V global
+        const bool sr = strong_rows(m, it);
+        const int parts = sr ? item_parts(it) : 1;
+        const int64_t kp = m->d.pair_id;
         switch (it.kind) {
         case IT_MATRIX:
         case IT_CONV_FWD:
         case IT_CONV_GW:
-            job(PJ_PAIR, {TAG_U0, TAG_U1}, cid, it.U.n, {it.U.p[0], it.U.p[1]});
-            job(PJ_PAIR, {TAG_V0, TAG_V1}, cid, it.V.n, {it.V.p[0], it.V.p[1]});
-            job(PJ_SINGLE, {TAG_Z0}, cid, it.Z.n, {it.Z.p[0]});
+            job(PJ_PAIR, {TAG_U0, TAG_U1}, cid, it.U.n, {it.U.p[0], it.U.p[1]}, sr ? kp * it.U.n / 8 : 0);
+            job(PJ_PAIR, {TAG_V0, TAG_V1}, cid, it.V.n, {it.V.p[0], it.V.p[1]}, 0);
+            job(PJ_SINGLE, {TAG_Z0}, cid, it.Z.n, {it.Z.p[0]}, sr ? kp * it.Z.n / 8 : 0);
             if (it.kind == IT_MATRIX && !m->ctx->use_tc(it.M, it.K, it.N) && it.M * it.N > 0) {
                 ClJob<DealerOps<T>> g{};
                 g.ops.U0 = it.U.p[0]; g.ops.U1 = it.U.p[1]; g.ops.V0 = it.V.p[0]; g.ops.V1 = it.V.p[1];
@@ -505,21 +535,30 @@ static psml_status build_plan(psml_model_s *m, int pool, bool infer_only) {
                 P.rest.push_back((int)k);
             }
             break;
-        case IT_HAD:
-            job(PJ_HAD, {TAG_U0, TAG_U1, TAG_V0, TAG_V1, TAG_Z0}, cid, it.n,
-                {it.U.p[0], it.U.p[1], it.V.p[0], it.V.p[1], it.Z.p[0], it.Z.p[1]});
-            break;
-        case IT_MSB: {   // the reduced prefix's 3 AND groups + the daBit (R27)
-            T *m0 = it.mat.p[0], *m1 = it.mat.p[1];
-            const int64_t n = it.n;
-            for (int g = 0; g < 3; ++g) {
-                const int64_t o = (int64_t)g * 3 * n;
-                job(PJ_AND, {tag4('a', '0', g), tag4('a', '1', g), tag4('b', '0', g), tag4('b', '1', g), tag4('c', '0', g)},
-                    cid, n, {m0 + o, m1 + o, m0 + o + n, m1 + o + n, m0 + o + 2 * n, m1 + o + 2 * n});
-                pjr.back().mask = msb_group_mask(64, g);
+        case IT_HAD: {
+            const int64_t per = it.n / parts;
+            for (int h = 0; h < parts; ++h) {
+                const int64_t q = h * per;   // local part h <- global part h, this pair's rows
+                job(PJ_HAD, {TAG_U0, TAG_U1, TAG_V0, TAG_V1, TAG_Z0}, cid, per,
+                    {it.U.p[0] + q, it.U.p[1] + q, it.V.p[0] + q, it.V.p[1] + q, it.Z.p[0] + q, it.Z.p[1] + q},
+                    sr ? strong_elem0(m, per, h) / 8 : 0);
             }
-            const int64_t o = (int64_t)9 * n;
-            job(PJ_DABIT, {TAG_R0, TAG_R1, TAG_RA}, cid, n, {m0 + o, m1 + o, m0 + o + n, m1 + o + n});
+            break;
+        }
+        case IT_MSB: {   // the reduced prefix's 3 AND groups + the daBit (R27); planes of n
+            T *m0 = it.mat.p[0], *m1 = it.mat.p[1];
+            const int64_t n = it.n, per = n / parts;
+            for (int h = 0; h < parts; ++h) {
+                const int64_t q = h * per, bo = sr ? strong_elem0(m, per, h) / 8 : 0;
+                for (int g = 0; g < 3; ++g) {
+                    const int64_t o = (int64_t)g * 3 * n + q;
+                    job(PJ_AND, {tag4('a', '0', g), tag4('a', '1', g), tag4('b', '0', g), tag4('b', '1', g), tag4('c', '0', g)},
+                        cid, per, {m0 + o, m1 + o, m0 + o + n, m1 + o + n, m0 + o + 2 * n, m1 + o + 2 * n}, bo);
+                    pjr.back().mask = msb_group_mask(64, g);
+                }
+                const int64_t o = (int64_t)9 * n + q;
+                job(PJ_DABIT, {TAG_R0, TAG_R1, TAG_RA}, cid, per, {m0 + o, m1 + o, m0 + o + n, m1 + o + n}, bo);
+            }
             break;
         }
         case IT_FSS:
@@ -582,6 +621,8 @@ static psml_status deal_prg_launch(psml_model_s *m, const DealPlan &P, int j0, i
 // material is ready early; s joins s2 before returning.
 static psml_status deal_pool(psml_model_s *m, int pool, uint32_t step, bool infer_only, cudaStream_t s,
                              cudaStream_t s2 = nullptr) {
+    if (m->d.strong_pairs > 1 && !fused_deal())
+        return fail(PSML_ERR_UNSUPPORTED, "strong scaling: the row-sliced material needs the fused dealer");
     if (!fused_deal() || m->d.mask_reuse) {   // mask reuse: the backward triplets copy forward masks
         for (auto &it : m->items[pool]) {
             if (infer_only && !it.fwd) continue;
@@ -1547,6 +1588,13 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
     }
     if (desc->mask_reuse && desc->kind != PSML_LINREG && desc->kind != PSML_LOGREG && desc->kind != PSML_MLP)
         return fail(PSML_ERR_UNSUPPORTED, "mask_reuse: linear / logistic regression and MLP");
+    if (desc->strong_pairs < 0 || desc->strong_pairs > 256) return fail(PSML_ERR_INVALID, "strong_pairs in [0, 256]");
+    if (desc->strong_pairs > 1) {   // strong-scaling dealer layout (R28)
+        if ((int64_t)desc->pair_id >= desc->strong_pairs) return fail(PSML_ERR_INVALID, "strong scaling: pair_id < strong_pairs");
+        if (desc->batch % 8) return fail(PSML_ERR_SHAPE, "strong scaling: batch must be a multiple of 8");
+        if (desc->kind == PSML_CNN || desc->mask_reuse)
+            return fail(PSML_ERR_UNSUPPORTED, "strong scaling: linear / logistic regression, MLP, SVM, RNN without mask_reuse");
+    }
     if (desc->weight_decay_shift < 0 || desc->weight_decay_shift >= 64)
         return fail(PSML_ERR_INVALID, "weight_decay_shift must be in [0, 64)");
     for (int l = 0; l < m->nl; ++l) {
@@ -1877,24 +1925,36 @@ psml_status psml_secure_train_step(psml_model m, const void *const X[2], const v
     return psml_train_apply_update(m, 0, stream);
 }
 
-// log2 of a data-parallel group size (the update's extra truncation bits); sizes must be 2^k
-static std::pair<psml_status, int> dp_shift(psml_dp dp) {
+// The party's data-parallel group: its size n and the update's extra truncation bits -- log2(n)
+// when every pair trains its own batch (weak scaling; n = 2^k), 0 under strong scaling (the sum
+// over the strong_pairs pairs IS the global-batch gradient, R28)
+struct DpGroup {
+    psml_status st;
+    int32_t n;
+    int shift;
+};
+static DpGroup dp_group(const psml_model_s *m, psml_dp dp) {
     int32_t n = 1;
-    if (dp && psml_dp_size(dp, &n) != PSML_OK) return {PSML_ERR_INVALID, 0};
+    if (dp && psml_dp_size(dp, &n) != PSML_OK) return {PSML_ERR_INVALID, 0, 0};
+    if (m->d.strong_pairs > 1) {
+        if (n != m->d.strong_pairs)
+            return {fail(PSML_ERR_INVALID, "strong scaling: the data-parallel group must hold strong_pairs ranks"), n, 0};
+        return {PSML_OK, n, 0};
+    }
     int sh = 0;
     while ((1 << sh) < n) ++sh;
-    if ((1 << sh) != n) return {fail(PSML_ERR_INVALID, "data-parallel group size must be a power of two"), 0};
-    return {PSML_OK, sh};
+    if ((1 << sh) != n) return {fail(PSML_ERR_INVALID, "data-parallel group size must be a power of two"), n, 0};
+    return {PSML_OK, n, sh};
 }
 
 // split deployment: all-reduce this party's untruncated gradient share over its data-parallel
 // group, then update its master / forward weight shares
 static psml_status party_reduce_update(psml_model_s *m, int party, psml_dp dp, cudaStream_t s) {
-    auto sh = dp_shift(dp);
-    PSML_TRY(sh.first);
-    if (dp && sh.second > 0)
+    const DpGroup g = dp_group(m, dp);
+    PSML_TRY(g.st);
+    if (dp && g.n > 1)
         PSML_TRY(psml_dp_allreduce(dp, m->grad_base + (int64_t)party * m->grad_words, m->grad_words, 64, (psml_stream)s));
-    return psml_party_apply_update(m, party, sh.second, (psml_stream)s);
+    return psml_party_apply_update(m, party, g.shift, (psml_stream)s);
 }
 
 // One captured step for online pool `pool`.  Non-pipelined: [dealer(pool)] -> online -> [update].
@@ -2019,7 +2079,7 @@ psml_status psml_party_capture_step(psml_model m, int32_t party, psml_xport x, p
     if (!m || !x) return fail(PSML_ERR_INVALID, "null model or transport");
     if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
     PSML_TRY(check_ptrs({X_i, Y_i}));
-    if (dp) PSML_TRY(dp_shift(dp).first);
+    if (dp) PSML_TRY(dp_group(m, dp).st);
     const void *X[2] = {nullptr, nullptr}, *Y[2] = {nullptr, nullptr};
     X[party] = X_i;
     Y[party] = Y_i;
@@ -2228,7 +2288,7 @@ psml_status psml_party_train_step(psml_model m, int32_t party, psml_xport x, psm
                                   const void *Y_i, uint32_t step_id, psml_stream stream) {
     PSML_CTX_OPTS(m ? m->ctx : nullptr);
     PSML_TRY(psml_party_forward_backward(m, party, x, X_i, Y_i, step_id, stream));
-    if (dp) PSML_TRY(dp_shift(dp).first);
+    if (dp) PSML_TRY(dp_group(m, dp).st);
     return party_reduce_update(m, party, dp, (cudaStream_t)stream);
 }
 

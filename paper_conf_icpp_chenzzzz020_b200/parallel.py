@@ -32,6 +32,16 @@ def dp_update_shift(world):
     return s
 
 
+def strong_rows(pair, n_pairs, global_batch):
+    """Rows of a global minibatch trained by pair `pair` of `n_pairs` under strong scaling
+    (R28): [pair b, (pair + 1) b) with b = global_batch / n_pairs, a multiple
+    of 8 (the row-sliced dealer streams start on ChaCha20 block boundaries)."""
+    b = global_batch // n_pairs if n_pairs > 0 else 0
+    if n_pairs <= 0 or b * n_pairs != global_batch or b % 8:
+        raise ValueError(f"global batch {global_batch} does not split into {n_pairs} pairs of 8k rows")
+    return slice(pair * b, (pair + 1) * b)
+
+
 def pair_rows(step, pair, n_pairs, batch, n_rows):
     """First row of minibatch `step` for pair `pair` of `n_pairs` (matches synth.batch)."""
     return ((step * n_pairs + pair) * batch) % (n_rows - batch + 1)

@@ -84,7 +84,8 @@ class ModelDesc(ctypes.Structure):
                 ("pair_id", u32), ("cnn_c", i32), ("cnn_h", i32), ("cnn_w", i32), ("cnn_k", i32),
                 ("cnn_cout", i32), ("cnn_hidden", i32), ("cnn_classes", i32),
                 ("fwd_frac_bits", i32 * 8), ("compare", i32), ("weight_decay_shift", i32),
-                ("rnn_steps", i32), ("mask_reuse", i32), ("deal_role", i32)]
+                ("rnn_steps", i32), ("mask_reuse", i32), ("deal_role", i32),
+                ("strong_pairs", i32)]
 
 
 # psml_exchange_fn (include/psml.h): (user, n, send[], recv[], bytes[], stream) -> 0 on success
@@ -598,7 +599,7 @@ class Model:
     def __init__(self, ctx, kind, dims=None, batch=128, lr_shift=14, master_frac_bits=27,
                  dealer_seed=0x50534D4C + 2, pair_id=0, cnn=(3, 32, 32, 5, 16, 64, 10),
                  fwd_frac_bits=None, compare=0, weight_decay_shift=0, rnn_steps=0, deal_role=0,
-                 mask_reuse=False):
+                 mask_reuse=False, strong_pairs=0):
         d = ModelDesc()
         d.kind = kind
         dims = list(dims or ([784, 1] if kind in (LINREG, LOGREG, SVM) else [784, 128, 128, 10]))
@@ -615,6 +616,7 @@ class Model:
         d.rnn_steps = rnn_steps                       # RNN sequence length (R25)
         d.deal_role = deal_role                       # 0 dealer, 1/2 party 0/1 dealing for itself (R23)
         d.mask_reuse = 1 if mask_reuse else 0         # forward/backward mask reuse (R26)
+        d.strong_pairs = strong_pairs                 # strong-scaling dealer layout
         self.ctx, self.desc, self.kind = ctx, d, kind
         h = vp()
         _call("psml_model_create", ctx.handle, ctypes.byref(d), ctypes.byref(h))

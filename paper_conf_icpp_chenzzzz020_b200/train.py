@@ -41,20 +41,23 @@ class SecureTrainer:
 
     def __init__(self, task, W_init, batch=128, pair_id=0, dims=None, backend=0,
                  frac_bits=13, master_frac_bits=27, lr_shift=14, compare="a2b", dealer_seed=DEALER_SEED,
-                 deal_role=0, w_shares=None, mask_reuse=False):
+                 deal_role=0, w_shares=None, mask_reuse=False, strong_pairs=0):
         self.task = task
         self.ctx = psml.Ctx(l=64, frac_bits=frac_bits, backend=backend)
         self.ring = self.ctx.ring
         self.master_ring = psml.Ring(64, master_frac_bits)
         self.pair_id = pair_id
         self.batch = batch
+        # strong scaling (R28): strong_pairs pairs share one global batch of
+        # strong_pairs * batch rows; this pair trains rows [pair_id * batch, (pair_id + 1) * batch)
+        self.strong_pairs = strong_pairs
         rnn = RNN_SHAPE if task == "rnn" else {}
         self.model = psml.Model(self.ctx, KINDS[task], dims=dims or rnn.get("dims"), batch=batch, lr_shift=lr_shift,
                                 rnn_steps=rnn.get("rnn_steps", 0),
                                 master_frac_bits=master_frac_bits, dealer_seed=dealer_seed, deal_role=deal_role,
                                 pair_id=pair_id, fwd_frac_bits=FWD_BITS.get(task),
                                 compare={"a2b": 0, "fss": 1}[compare], weight_decay_shift=WD_SHIFT.get(task, 0),
-                                mask_reuse=mask_reuse)
+                                mask_reuse=mask_reuse, strong_pairs=strong_pairs)
         for layer, W in enumerate(W_init):
             if w_shares is not None:   # shares handed over by the client: w_shares[layer] = (Wm_0, Wm_1)
                 self.model.set_master(layer, w_shares[layer])
@@ -156,7 +159,16 @@ class SecureTrainer:
         self.model.forward_backward(Xs, Ys, step)
         world = dist.get_world_size(group) if dist.is_initialized() else 1
         ring_allreduce_(self.grad_tensor(), group)
-        self.model.apply_update(extra_shift=dp_update_shift(world))
+        self.model.apply_update(extra_shift=self.update_shift(world))
+
+    def update_shift(self, world):
+        """Extra truncation of the summed gradient: log2(pairs) when each pair trains its own
+        batch (weak scaling); 0 under strong scaling, where the sum IS the global-batch gradient."""
+        if self.strong_pairs > 1:
+            if world != self.strong_pairs:
+                raise ValueError(f"strong scaling over {self.strong_pairs} pairs, all-reduce over {world}")
+            return 0
+        return dp_update_shift(world)
 
     def last_yhat(self):
         """Prediction shares of the last step as two uint64 views of model-owned memory."""
@@ -232,7 +244,7 @@ class PartyTrainer(SecureTrainer):
         ptr, words = self.model.grads()
         g = _wrap_device_ptr(ptr + 8 * words * self.party, words)
         ring_allreduce_(g, dp_group)
-        self.model.party_apply_update(self.party, extra_shift=dp_update_shift(dp_world))
+        self.model.party_apply_update(self.party, extra_shift=self.update_shift(dp_world))
 
     def capture_party(self, pipelined=True):
         """Capture this party's whole step (dealer [pipelined], online phase with its exchanges,

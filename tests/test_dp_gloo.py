@@ -90,6 +90,59 @@ def test_dp_two_pairs_gloo_matches_single_process_sum(tmp_path, task):
         assert big.tolist() == [(2 ** 63 - 1) * 2 - 1, 2 ** 64 - 2, 10]
 
 
+def _strong_worker(rank, world, port, task, outdir):
+    """Pair `rank` of a strong-scaling group (R28): rows [rank b, (rank + 1) b)
+    of the global batch, row-sliced material, gradient all-reduce over gloo, no extra shift."""
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import synth
+    from oracle import protocol as OP
+    from paper_conf_icpp_chenzzzz020_b200.parallel import ring_allreduce_, strong_rows
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    m = OP.Model(task, synth.init_weights(task))
+    for step in range(2):
+        X, Y = synth.batch(task, step)
+        Xs, Ys = OP.share_batch(X, Y, step)          # the client shares the global batch
+        r = strong_rows(rank, world, X.shape[0])     # ... and this pair receives its rows
+        grads, _ = OP.forward_backward(m, (Xs[0][r], Xs[1][r]), (Ys[0][r], Ys[1][r]), step, OP.Strong(rank, world))
+        flat = torch.from_numpy(_flatten(grads))
+        ring_allreduce_(flat)
+        OP.apply_update(m, _unflatten(flat.numpy(), grads), n_pairs=1)
+    np.savez(os.path.join(outdir, f"strong{rank}.npz"), *[w for pair in m.Wm for w in pair])
+    dist.destroy_process_group()
+
+
+def test_strong_dp_two_pairs_gloo_matches_oracle():
+    import tempfile
+
+    import synth
+    from oracle import protocol as OP
+    world, task = 2, "mlp"
+    with tempfile.TemporaryDirectory() as d:
+        mp.spawn(_strong_worker, args=(world, _free_port(), task, d), nprocs=world, join=True)
+        m = OP.Model(task, synth.init_weights(task))
+        for step in range(2):
+            X, Y = synth.batch(task, step)
+            Xs, Ys = OP.share_batch(X, Y, step)
+            grads, _ = OP.strong_forward_backward(m, Xs, Ys, step, world)
+            OP.apply_update(m, grads, n_pairs=1)
+        want = [w for pair in m.Wm for w in pair]
+        for r in range(world):
+            got = np.load(os.path.join(d, f"strong{r}.npz"))
+            for i, w in enumerate(want):
+                assert np.array_equal(got[f"arr_{i}"], w), (r, i)
+
+
+def test_strong_rows():
+    from paper_conf_icpp_chenzzzz020_b200.parallel import strong_rows
+    assert [strong_rows(k, 4, 128) for k in range(4)] == [slice(0, 32), slice(32, 64), slice(64, 96), slice(96, 128)]
+    with pytest.raises(ValueError):
+        strong_rows(0, 3, 128)        # 128 rows do not split into 3 pairs
+    with pytest.raises(ValueError):
+        strong_rows(0, 32, 128)       # 4 rows per pair: not a multiple of 8 (ChaCha20 block slices)
+
+
 def test_dp_update_shift_and_rows():
     from paper_conf_icpp_chenzzzz020_b200.parallel import dp_update_shift, pair_rows
     import synth
