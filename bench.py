@@ -875,6 +875,54 @@ def cfg5_sweep(ns):
 
 
 
+def cfg5_sharded(ns, world, rank):
+    """Config 5 over `world` GPUs (bench.py --sweep under torchrun): M-row sharding of the n^3
+    product over data-parallel pairs: pair r holds rows [r n / world, (r + 1) n / world)
+    of A (and of U, Z: psml_triplet_gen_rows) and the whole B (and V), computes its C rows with no
+    cross-pair collective; the plain ring GEMM and the co-resident Beaver secure matmul are both
+    timed per rank with CUDA events (barrier + synchronize around), the max over ranks taken, and
+    the aggregate useful TOPS = the whole n^3 product's limb ops / that time.  Rank 0 checks its
+    row block bit-exactly against the CPU oracle for n <= 1024.  One JSON line per (n, l) on rank 0."""
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+    from oracle import core as orc
+    from paper_conf_icpp_chenzzzz020_b200 import psml
+    for n in ns:
+        if n % world:
+            continue
+        m = n // world
+        r0 = rank * m
+        for l in (64, 32):
+            pairs = 36 if l == 64 else 10
+            ring = psml.Ring(l, 13)
+            A = psml.prg_fill(ring, 1, psml.tag("bA"), 0, m * n, offset=r0 * n).view(m, n)   # this pair's rows of A
+            B = psml.prg_fill(ring, 1, psml.tag("bB"), 0, n * n).view(n, n)
+            C = psml.empty(0, l, (m, n))
+            reps = 5 if n >= 4096 else 10
+            ctx = psml.Ctx(l=l)
+            dist.barrier()
+            ms = max_over_ranks(tev(lambda: psml.ring_gemm(ctx, A, B, out=C), reps), world)
+            row = {"n": n, "l": l, "gpus": world, "sharding": "M rows over pairs (no cross-pair collective)",
+                   "rows_per_gpu": m, "gemm_ms": ms, "gemm_useful_tops_aggregate": pairs * 2.0 * n ** 3 / ms / 1e9}
+            As = psml.share(ring, 7, 1, A)
+            Bs = psml.share(ring, 7, 2, B)
+            U, V, Z = psml.triplet_gen_rows(ctx, 3, 0, n, r0, m, n, n)
+            Cs = psml.empty_pair((m, n), l)
+            dist.barrier()
+            ms = max_over_ranks(tev(lambda: psml.secure_matmul(ctx, As, Bs, U, V, Z, m, n, n, trunc=13, out=Cs),
+                                    reps), world)
+            row["beaver_ms"] = ms
+            row["beaver_useful_tops_aggregate"] = 2 * 2 * pairs * 2.0 * n ** 3 / ms / 1e9
+            if n <= 1024 and rank == 0:
+                W = orc.ring_matmul(A.cpu().numpy().astype(np.uint64), B.cpu().numpy().astype(np.uint64), l)
+                row["bitexact_vs_oracle_rank0_rows"] = bool(np.array_equal(C.cpu().numpy().astype(np.uint64), W))
+            ctx.close()
+            if rank == 0:
+                print(json.dumps(row), flush=True)
+            torch.cuda.synchronize()
+
+
 def cpu_model():
     try:
         for line in open("/proc/cpuinfo"):
@@ -1034,7 +1082,12 @@ def main():
     if args.sweep:
         from paper_conf_icpp_chenzzzz020_b200 import build
         build.build()
-        cfg5_sweep([int(x) for x in args.sweep.split(",")])
+        ns = [int(x) for x in args.sweep.split(",")]
+        if int(os.environ.get("WORLD_SIZE", "1")) > 1:
+            world, rank, _ = dist_setup(args)
+            cfg5_sharded(ns, world, rank)
+        else:
+            cfg5_sweep(ns)
         return
     world = int(os.environ.get("WORLD_SIZE", "1"))
     if args.deployment == "split" or (args.deployment == "auto" and world >= 2):

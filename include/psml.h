@@ -169,6 +169,16 @@ psml_status psml_reconstruct(psml_ring ring, const void *x0, const void *x1, int
 psml_status psml_triplet_gen(psml_ctx ctx, uint64_t seed, uint64_t call_id, int64_t M, int64_t K,
                              int64_t N, void *const U[2], void *const V[2], void *const Z[2],
                              psml_stream stream);
+/* Rows [row0, row0 + M) of the M_total x K by K x N triplet psml_triplet_gen(seed, call_id,
+ * M_total, K, N) would deal: U_i rows (elements row0*K .. of the "U0"/"U1" streams), the WHOLE V_i
+ * and Z_i rows (Z_0 elements row0*N .., Z_1 = U[rows] V - Z_0[rows]); bit-identical to slicing the
+ * full triplet.  The M-row sharding of a secure product over data-parallel pairs (SURVEY 8(e)
+ * config 5, R28): pair k deals its own rows, every pair opens the same F = B - V.
+ * U_i: M x K, V_i: K x N, Z_i: M x N (device, caller-owned).  PSML_ERR_SHAPE unless
+ * 0 <= row0, M > 0 and row0 + M <= M_total. */
+psml_status psml_triplet_gen_rows(psml_ctx ctx, uint64_t seed, uint64_t call_id, int64_t M_total, int64_t row0,
+                                  int64_t M, int64_t K, int64_t N, void *const U[2], void *const V[2],
+                                  void *const Z[2], psml_stream stream);
 /* Elementwise (Hadamard) triplet of n elements: same streams, Z_1 = (U_0+U_1)(V_0+V_1) - Z_0. */
 psml_status psml_hadamard_triplet_gen(psml_ring ring, uint64_t seed, uint64_t call_id, int64_t n,
                                       void *const U[2], void *const V[2], void *const Z[2],
@@ -439,6 +449,13 @@ psml_status psml_model_step_graph(psml_model model, uint32_t step_id, psml_strea
  * host buffers must stay valid until it completes.  PSML_ERR_STATE without a captured step. */
 psml_status psml_model_step_host(psml_model model, const uint8_t *q, const void *y, int32_t y_kind,
                                  uint64_t share_seed, uint32_t step_id, void *yhat_host, psml_stream stream);
+/* One whole step from DEVICE plaintext (the client's batch already in HBM): encodes and shares
+ * X (batch x features float64, device) and Y (batch x d_L float64, device) into the captured X/Y
+ * buffers in ONE launch -- bit-identical to psml_encode_share with the share ids of
+ * psml_model_step_host -- then replays the captured step (psml_model_step_graph, same
+ * preconditions).  Co-resident captured step only; asynchronous on `stream`. */
+psml_status psml_model_step_device(psml_model model, const double *X, const double *Y, uint64_t share_seed,
+                                   uint32_t step_id, psml_stream stream);
 /* Number of kernel nodes in the captured step graph (launch accounting for bench.py). */
 psml_status psml_model_graph_nodes(psml_model model, int64_t *n);
 /* Secure inference (the forward half): Yhat[i]: batch x d_L.  Needs

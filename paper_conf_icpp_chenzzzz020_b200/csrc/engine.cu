@@ -452,17 +452,26 @@ psml_status psml_reconstruct(psml_ring ring, const void *x0, const void *x1, int
 // ------------------------------------------------------------------------------------------------
 // dealer
 // ------------------------------------------------------------------------------------------------
+// rows [row0, row0 + M) of the triplet (row0 = 0: the whole M x K by K x N triplet)
 template <typename T>
-static psml_status triplet_gen_t(Ctx *c, uint64_t seed, uint64_t cid, int64_t M, int64_t K, int64_t N,
+static psml_status triplet_gen_t(Ctx *c, uint64_t seed, uint64_t cid, int64_t row0, int64_t M, int64_t K, int64_t N,
                                  void *const U[2], void *const V[2], void *const Z[2], cudaStream_t s) {
     const DealSeeds S = dealer_seeds(seed);
-    dealer_pair_kernel<T><<<grid_for(M * K / 8 + 1, 256), 256, 0, s>>>(dkey(S, TAG_U0, cid), dkey(S, TAG_U1, cid), M * K,
-                                                                       (T *)U[0], (T *)U[1], nullptr);
-    PSML_LAUNCH_CHECK();
+    if (row0 == 0) {
+        dealer_pair_kernel<T><<<grid_for(M * K / 8 + 1, 256), 256, 0, s>>>(dkey(S, TAG_U0, cid), dkey(S, TAG_U1, cid),
+                                                                           M * K, (T *)U[0], (T *)U[1], nullptr);
+        PSML_LAUNCH_CHECK();
+    } else {   // a row block: the U streams from element row0 * K (any alignment)
+        for (int i = 0; i < 2; ++i) {
+            prg_kernel<T, 0><<<grid_for(M * K / 8 + 2, 256), 256, 0, s>>>(dkey(S, i ? TAG_U1 : TAG_U0, cid), row0 * K,
+                                                                          M * K, (T *)U[i], nullptr, nullptr);
+            PSML_LAUNCH_CHECK();
+        }
+    }
     dealer_pair_kernel<T><<<grid_for(K * N / 8 + 1, 256), 256, 0, s>>>(dkey(S, TAG_V0, cid), dkey(S, TAG_V1, cid), K * N,
                                                                        (T *)V[0], (T *)V[1], nullptr);
     PSML_LAUNCH_CHECK();
-    prg_kernel<T, 0><<<grid_for(M * N / 8 + 2, 256), 256, 0, s>>>(dkey(S, TAG_Z0, cid), 0, M * N, (T *)Z[0],
+    prg_kernel<T, 0><<<grid_for(M * N / 8 + 2, 256), 256, 0, s>>>(dkey(S, TAG_Z0, cid), row0 * N, M * N, (T *)Z[0],
                                                                   nullptr, nullptr);
     PSML_LAUNCH_CHECK();
     // Z = (U0+U1)(V0+V1) on the tensor cores where it pays, else the CUDA-core ring GEMM
@@ -491,8 +500,23 @@ psml_status psml_triplet_gen(psml_ctx ctx, uint64_t seed, uint64_t call_id, int6
     if (!U || !V || !Z) return fail(PSML_ERR_INVALID, "null pair array");
     PSML_TRY(check_ptrs({U[0], U[1], V[0], V[1], Z[0], Z[1]}));
     cudaStream_t s = (cudaStream_t)stream;
-    if (c->ring.l == 64) return triplet_gen_t<uint64_t>(c, seed, call_id, M, K, N, U, V, Z, s);
-    return triplet_gen_t<uint32_t>(c, seed, call_id, M, K, N, U, V, Z, s);
+    if (c->ring.l == 64) return triplet_gen_t<uint64_t>(c, seed, call_id, 0, M, K, N, U, V, Z, s);
+    return triplet_gen_t<uint32_t>(c, seed, call_id, 0, M, K, N, U, V, Z, s);
+}
+
+psml_status psml_triplet_gen_rows(psml_ctx ctx, uint64_t seed, uint64_t call_id, int64_t M_total, int64_t row0,
+                                  int64_t M, int64_t K, int64_t N, void *const U[2], void *const V[2],
+                                  void *const Z[2], psml_stream stream) {
+    PSML_CTX_OPTS(ctx);
+    if (!ctx) return fail(PSML_ERR_INVALID, "ctx is null");
+    Ctx *c = reinterpret_cast<Ctx *>(ctx);
+    if (M <= 0 || K <= 0 || N <= 0 || row0 < 0 || row0 + M > M_total)
+        return fail(PSML_ERR_SHAPE, "rows [row0, row0 + M) must lie in [0, M_total); M, K, N > 0");
+    if (!U || !V || !Z) return fail(PSML_ERR_INVALID, "null pair array");
+    PSML_TRY(check_ptrs({U[0], U[1], V[0], V[1], Z[0], Z[1]}));
+    cudaStream_t s = (cudaStream_t)stream;
+    if (c->ring.l == 64) return triplet_gen_t<uint64_t>(c, seed, call_id, row0, M, K, N, U, V, Z, s);
+    return triplet_gen_t<uint32_t>(c, seed, call_id, row0, M, K, N, U, V, Z, s);
 }
 
 psml_status psml_hadamard_triplet_gen(psml_ring ring, uint64_t seed, uint64_t call_id, int64_t n, void *const U[2],

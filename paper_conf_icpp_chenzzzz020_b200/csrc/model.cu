@@ -30,6 +30,8 @@ enum { OP_FWD = 0, OP_GRADW = 1, OP_GRADIN = 2, OP_RELU_MSB = 3, OP_EQ9_MSB = 4,
 enum ItemKind { IT_MATRIX, IT_CONV_FWD, IT_CONV_GW, IT_HAD, IT_MSB, IT_FSS };   // IT_FSS: DCF material (R22)
 
 __global__ void set_word_kernel(uint32_t *p, uint32_t v) { *p = v; }
+// last node of a pipelined graph's dealer branch: the next consecutive replay's step word
+__global__ void advance_word_kernel(uint32_t *p) { *p += 1; }
 
 // Co-resident Beaver matmuls run the explicit mask round then the GEMM that opens E/F (default:
 // measured faster inside the CUDA graph, 338K vs 328K samples/s) or fuse the mask into the GEMM's
@@ -115,6 +117,8 @@ struct psml_model_s {
     bool dealt_full[2] = {false, false};
     bool grads_ready = false;
     uint32_t *step_dev = nullptr;      // device copy of the step number (dealer call ids)
+    int64_t word_next = -1;            // value *step_dev holds once the last enqueued pipelined
+                                       // replay completes (it advances the word itself); -1 unknown
     cudaGraphExec_t graph[2] = {nullptr, nullptr};  // captured step(s) (psml_model_capture_step)
     int graph_flags = 0;
     int64_t graph_kernels = 0;
@@ -988,6 +992,8 @@ static psml_status deal_fork_point(psml_model_s *m, cudaStream_t s, bool force =
     const psml_status st = deal_pool(m, pool, 0, false, m->side, deal_s2(m));
     m->deal_alone = false;
     PSML_TRY(st);
+    advance_word_kernel<<<1, 1, 0, m->side>>>(m->step_dev);   // every reader of the word is done
+    PSML_LAUNCH_CHECK();
     PSML_CUDA_TRY(cudaEventRecord(m->ev_join, m->side));
     return PSML_OK;
 }
@@ -1770,6 +1776,7 @@ psml_status psml_model_deal(psml_model m, uint32_t step_id, int32_t infer_only, 
     const int pool = (int)(step_id & 1);
     set_word_kernel<<<1, 1, 0, s>>>(m->step_dev, step_id);
     PSML_LAUNCH_CHECK();
+    m->word_next = -1;
     PSML_TRY(deal_pool(m, pool, step_id, infer_only != 0, s));
     m->dealt_step[pool] = step_id;
     m->dealt_full[pool] = !infer_only;
@@ -1983,6 +1990,7 @@ static psml_status capture_one(psml_model_s *m, int pool, const T *const X[2], c
         m->deal_stage = 0;
         if (st == PSML_OK && m->deal_after == 0) {
             st = deal_pool(m, 1 - pool, 0, false, m->side, deal_s2(m));
+            if (st == PSML_OK) advance_word_kernel<<<1, 1, 0, m->side>>>(m->step_dev);
             if (st == PSML_OK && cudaEventRecord(m->ev_join, m->side) != cudaSuccess)
                 st = fail(PSML_ERR_CUDA, "graph join record failed");
         } else {
@@ -2047,6 +2055,7 @@ static psml_status capture_common(psml_model m, const void *const X[2], const vo
             m->graph[g] = nullptr;
         }
     const int prof = g_prof_cls.exchange(-1);   // no profiling events inside the graphs
+    m->word_next = -1;
     psml_status st = PSML_OK;
     // one graph per dealer pool, except when the graph deals its own pool 0 (flags bit 0 only)
     // or replays one pool on purpose (bit 3, benchmark-only material reuse)
@@ -2096,7 +2105,8 @@ psml_status psml_party_capture_step(psml_model m, int32_t party, psml_xport x, p
 // (one-hot) or float64 labels -- the same words as psml_encode_share_u8 / _onehot / encode_share.
 struct ClientJob {
     PrgKey kx, ky;
-    const uint8_t *q;
+    const uint8_t *q;     // X as 8-bit pixels (x = q / 255), or
+    const double *xf;     // X as float64 (q == nullptr)
     const uint8_t *ycls;
     const double *yf;
     int64_t nx, ny, classes;
@@ -2115,7 +2125,7 @@ __global__ void __launch_bounds__(128) client_share_kernel(const ClientJob j) {
             const int64_t e = b * 8 + t;
             if (e >= n) break;
             double x;
-            if (isx) x = (double)j.q[e] / 255.0;
+            if (isx) x = j.q ? (double)j.q[e] / 255.0 : j.xf[e];
             else if (j.ycls) x = (int64_t)j.ycls[e / j.classes] == e % j.classes ? 1.0 : 0.0;
             else x = j.yf[e];
             const uint64_t r = ((uint64_t)w[2 * t + 1] << 32) | w[2 * t];
@@ -2208,10 +2218,38 @@ psml_status psml_model_step_host(psml_model m, const uint8_t *q, const void *y, 
     return PSML_OK;
 }
 
+// features per input row: CNN C H W, RNN T D, else d_0
+static int64_t x_row(const psml_model_s *m) {
+    if (m->d.kind == PSML_CNN) return (int64_t)m->g.C * m->g.H * m->g.W;
+    if (m->d.kind == PSML_RNN) return (int64_t)m->rnn_T * m->rnn_D;
+    return m->dims[0];
+}
+
+psml_status psml_model_step_device(psml_model m, const double *X, const double *Y, uint64_t share_seed,
+                                   uint32_t step_id, psml_stream stream) {
+    PSML_CTX_OPTS(m ? m->ctx : nullptr);
+    if (!m || !X || !Y) return fail(PSML_ERR_INVALID, "null argument");
+    if (!m->graph[0] || !m->cap_X[0]) return fail(PSML_ERR_STATE, "no captured step: call psml_model_capture_step first");
+    if (m->cap_party >= 0) return fail(PSML_ERR_STATE, "psml_model_step_device serves the co-resident captured step");
+    PSML_TRY(check_ptrs({X, Y}));
+    cudaStream_t s = (cudaStream_t)stream;
+    const int64_t nx = m->B * x_row(m), ny = m->B * m->dims.back();
+    // client: encode + share X and Y into the captured buffers, one launch (R3, R11 share ids)
+    ClientJob cj{};
+    cj.kx = make_key(share_seed, TAG_SH, call_id(m->d.pair_id, step_id, 0, OP_SHARE, 0));
+    cj.ky = make_key(share_seed, TAG_SH, call_id(m->d.pair_id, step_id, 0, OP_SHARE, 1));
+    cj.xf = X; cj.nx = nx; cj.f = m->ctx->ring.frac_bits;
+    cj.yf = Y; cj.ny = ny; cj.classes = m->dims.back();
+    cj.x0 = (T *)m->cap_X[0]; cj.x1 = (T *)m->cap_X[1]; cj.y0 = (T *)m->cap_Y[0]; cj.y1 = (T *)m->cap_Y[1];
+    client_share_kernel<<<grid_for((nx + 7) / 8 + (ny + 7) / 8, 128), 128, 0, s>>>(cj);
+    PSML_LAUNCH_CHECK();
+    return psml_model_step_graph(m, step_id, stream);
+}
+
 psml_status psml_model_graph_nodes(psml_model m, int64_t *n) {
     PSML_CTX_OPTS(m ? m->ctx : nullptr);
     if (!m || !n) return fail(PSML_ERR_INVALID, "null argument");
-    *n = m->graph_kernels + 1;   // + the step-word kernel launched before each replay
+    *n = m->graph_kernels;   // (+ a step-word kernel before a replay only when the step sequence jumps)
     return PSML_OK;
 }
 
@@ -2230,9 +2268,15 @@ psml_status psml_model_step_graph(psml_model m, uint32_t step_id, psml_stream st
         return fail(PSML_ERR_STATE, "psml_model_deal(step_id) must have filled this step's pool (material is single-use)");
     if (reuse && (m->dealt_step[0] < 0 || !m->dealt_full[0]))
         return fail(PSML_ERR_STATE, "reuse graph: pool 0 was never dealt");
-    set_word_kernel<<<1, 1, 0, s>>>(m->step_dev, pipelined ? step_id + 1 : step_id);
-    PSML_LAUNCH_CHECK();
+    // the step word the graph's dealer reads: a pipelined replay advances it for the next
+    // consecutive step itself, so it is written from the host only when the sequence jumps
+    const uint32_t word = pipelined ? step_id + 1 : step_id;
+    if (!pipelined || m->word_next != (int64_t)word) {
+        set_word_kernel<<<1, 1, 0, s>>>(m->step_dev, word);
+        PSML_LAUNCH_CHECK();
+    }
     PSML_CUDA_TRY(cudaGraphLaunch(m->graph[(self_dealt || reuse) ? 0 : pool], s));
+    m->word_next = pipelined ? (int64_t)word + 1 : -1;
     g_launches.fetch_add((uint64_t)m->graph_kernels);   // the graph's kernels are our launches
     if (pipelined) {
         m->dealt_step[pool] = -1;                        // consumed

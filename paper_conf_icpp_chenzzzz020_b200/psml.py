@@ -114,6 +114,7 @@ _SIGS = {
     "psml_encode_share_u8": (i32, [Ring, u64, u64, vp, i64, ctypes.c_double, vp, vp, vp]),
     "psml_encode_share_onehot": (i32, [Ring, u64, u64, vp, i64, i64, vp, vp, vp]),
     "psml_triplet_gen": (i32, [vp, u64, u64, i64, i64, i64, P2, P2, P2, vp]),
+    "psml_triplet_gen_rows": (i32, [vp, u64, u64, i64, i64, i64, i64, i64, P2, P2, P2, vp]),
     "psml_hadamard_triplet_gen": (i32, [Ring, u64, u64, i64, P2, P2, P2, vp]),
     "psml_msb_material_words": (i64, [Ring, i64]),
     "psml_msb_dealer": (i32, [Ring, u64, u64, i64, P2, vp]),
@@ -143,6 +144,7 @@ _SIGS = {
     "psml_model_capture_step": (i32, [vp, P2, P2, i32, vp]),
     "psml_model_step_graph": (i32, [vp, u32, vp]),
     "psml_model_step_host": (i32, [vp, vp, vp, i32, u64, u32, vp, vp]),
+    "psml_model_step_device": (i32, [vp, vp, vp, u64, u32, vp]),
     "psml_model_graph_nodes": (i32, [vp, vp]),
     "psml_nccl_unique_id": (i32, [vp]),
     "psml_xport_nccl_create": (i32, [vp, i32, vp]),
@@ -409,6 +411,15 @@ def reconstruct(ring, x0, x1, stream=None):
 def triplet_gen(ctx, seed, call_id, M, K, N, stream=None):
     U, V, Z = empty_pair((M, K), ctx.l), empty_pair((K, N), ctx.l), empty_pair((M, N), ctx.l)
     _call("psml_triplet_gen", ctx.handle, seed, call_id, M, K, N, _pair(U), _pair(V), _pair(Z),
+          _stream(stream))
+    return U, V, Z
+
+
+def triplet_gen_rows(ctx, seed, call_id, M_total, row0, M, K, N, stream=None):
+    """Rows [row0, row0 + M) of triplet_gen(seed, call_id, M_total, K, N): U / Z row blocks and the
+    whole V (the M-row sharding of a secure product over pairs, R28)."""
+    U, V, Z = empty_pair((M, K), ctx.l), empty_pair((K, N), ctx.l), empty_pair((M, N), ctx.l)
+    _call("psml_triplet_gen_rows", ctx.handle, seed, call_id, M_total, row0, M, K, N, _pair(U), _pair(V), _pair(Z),
           _stream(stream))
     return U, V, Z
 
@@ -704,6 +715,13 @@ class Model:
 
     def step_graph(self, step, stream=None):
         _call("psml_model_step_graph", self.handle, step, _stream(stream))
+
+    def step_device(self, X, Y, share_seed, step, stream=None):
+        """psml_model_step_device: X, Y float64 device tensors (the batch in HBM); one launch
+        encodes and shares both into the captured buffers, then the captured step replays."""
+        _check(X, self.x_words, (torch.float64,), "step_device X")
+        _check(Y, self.y_words, (torch.float64,), "step_device Y")
+        _call("psml_model_step_device", self.handle, _ptr(X), _ptr(Y), share_seed, step, _stream(stream))
 
     def step_host(self, q, y, share_seed, step, yhat_host, stream=None):
         """psml_model_step_host: q uint8 pixels, y float64 labels or uint8 class indices, yhat_host

@@ -123,11 +123,16 @@ class SecureTrainer:
         return self.model.graph_nodes()
 
     def graph_step(self, X, Y, step):
-        """Client encode + share into the captured buffers, then replay the captured step."""
-        self._client_share(X, Y, step, outX=self.Xbuf, outY=self.Ybuf)
+        """Client encode + share into the captured buffers, then replay the captured step (float64
+        device batches: one library call, psml_model_step_device)."""
         if self.pipelined and self._next_dealt != step:
             self.model.deal(step)          # prime the pipeline (first step or a jump in step ids)
-        self.model.step_graph(step)
+        if (torch.is_tensor(X) and torch.is_tensor(Y) and X.is_cuda and Y.is_cuda and X.dtype == torch.float64
+                and Y.dtype == torch.float64):
+            self.model.step_device(X.contiguous(), Y.contiguous(), SHARE_SEED, step)
+        else:
+            self._client_share(X, Y, step, outX=self.Xbuf, outY=self.Ybuf)
+            self.model.step_graph(step)
         self._next_dealt = step + 1
 
     def graph_step_host(self, q, y, step, yhat_host):

@@ -114,6 +114,22 @@ def test_triplet_gen(P, orc, ctx, shape):
         assert np.array_equal(g, w)
 
 
+@pytest.mark.parametrize("M_total,cuts,K,N", [(100, (0, 37, 100), 33, 65), (4096, (0, 1024, 2048, 3072, 4096), 16, 8),
+                                               (9, (0, 1, 9), 1, 1)])
+def test_triplet_gen_rows_are_slices_of_the_full_triplet(P, orc, ctx, M_total, cuts, K, N):
+    """psml_triplet_gen_rows (M-row sharding, R28): row blocks (ragged, unaligned to
+    ChaCha20 blocks) equal the oracle's full triplet sliced; V is the whole V of every block."""
+    want = orc.triplet_gen(SEED + 2, 4242, M_total, K, N, ctx.l)
+    for r0, r1 in zip(cuts[:-1], cuts[1:]):
+        U, V, Z = P.triplet_gen_rows(ctx, SEED + 2, 4242, M_total, r0, r1 - r0, K, N)
+        got = pair_np(U) + pair_np(V) + pair_np(Z)
+        rows = slice(r0, r1)
+        for g, w, sliced in zip(got, want, (True, True, False, False, True, True)):
+            assert np.array_equal(g, w[rows] if sliced else w)
+    with pytest.raises(P.PsmlError):
+        P.triplet_gen_rows(ctx, SEED + 2, 4242, M_total, M_total - 1, 2, K, N)
+
+
 def test_hadamard_triplet_and_msb_material(P, orc, ctx):
     ring = ctx.ring
     for n in (1, 17, 5003):

@@ -100,6 +100,27 @@ def test_graph_replay_bitexact_vs_oracle(T, task, steps, pipelined):
     tr.close()
 
 
+@pytest.mark.parametrize("task", ["mlp", "logreg", "rnn"])
+def test_step_device_bitexact_vs_oracle_with_step_jumps(T, task):
+    """psml_model_step_device (device float64 batch: one share launch + the pipelined graph, whose
+    dealer branch advances the step word for the next consecutive replay) matches the oracle over
+    consecutive steps and after jumps in the step ids (the host rewrites the word)."""
+    Wi = synth.init_weights(task)
+    tr = T.SecureTrainer(task, Wi, backend=0)
+    om = OP.Model(task, Wi)
+    X, Y = synth.batch(task, 0)
+    tr.step(torch.from_numpy(X), torch.from_numpy(Y), 0)
+    OP.train_step(om, X, Y, 0)
+    tr.capture(pipelined=True)
+    for s in (1, 2, 3, 9, 10, 4, 5):
+        X, Y = synth.batch(task, s)
+        tr.graph_step(torch.from_numpy(X).cuda(), torch.from_numpy(Y).cuda(), s)
+        OP.train_step(om, X, Y, s)
+        torch.cuda.synchronize()
+        _compare_shares(tr, om)
+    tr.close()
+
+
 @pytest.mark.parametrize("task", ["mlp", "logreg", "cnn"])
 def test_step_host_bitexact_vs_oracle(T, task):
     """psml_model_step_host (host pixels + labels in, captured step, prediction shares out: the
