@@ -119,6 +119,10 @@ typedef struct {
     int32_t split_fused;   /* split deployment over a peer transport: 1 each activation is ONE
                               kernel with its 9 rounds' exchanges fused over peer memory, 0 one
                               kernel + one exchange per round                                   */
+    int32_t deal_on_launch; /* pipelined graph: 1 = the dealer branch forks as soon as every CTA of
+                              the first tcgen05 product is resident (a launch-completion edge),
+                              so the product's SMs are taken before the dealer's grids; 0 = after
+                              the deal_after-th online stage completes                          */
 } psml_options;
 psml_status psml_options_default(psml_options *out);
 psml_status psml_ctx_set_options(psml_ctx ctx, const psml_options *opts);

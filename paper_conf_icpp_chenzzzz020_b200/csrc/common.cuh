@@ -135,6 +135,10 @@ __host__ __device__ inline PrgKey make_key(uint64_t seed, uint32_t tag, uint64_t
 // The options of the context the current ABI call runs on (psml_options; a thread-local pointer
 // set for the duration of the call -- contexts are per host thread, include/psml.h).
 const psml_options &cur_opts();
+// A launch-completion event for the next tcgen05 product launch (psml_options.deal_on_launch:
+// the pipelined graph's dealer fork edge); take_launch_event returns and clears it.
+void arm_launch_event(cudaEvent_t e);
+cudaEvent_t take_launch_event();
 struct OptScope {
     const psml_options *prev;
     explicit OptScope(const psml_options *o);

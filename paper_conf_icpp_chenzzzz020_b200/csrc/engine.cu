@@ -291,8 +291,15 @@ psml_status psml_secure_matmul_party(psml_ctx ctx, const void *A_i, const void *
 }
 
 namespace psml {
-static const psml_options k_default_opts{0, 1, 0, 1, 1, 1, 1, 1, 1, 1, 0, 1, 1};
+static const psml_options k_default_opts{0, 1, 0, 1, 1, 1, 1, 1, 1, 1, 0, 1, 1, 0};
 static thread_local const psml_options *t_opts = nullptr;
+static thread_local cudaEvent_t t_launch_event = nullptr;
+void arm_launch_event(cudaEvent_t e) { t_launch_event = e; }
+cudaEvent_t take_launch_event() {
+    cudaEvent_t e = t_launch_event;
+    t_launch_event = nullptr;
+    return e;
+}
 const psml_options &cur_opts() { return t_opts ? *t_opts : k_default_opts; }
 OptScope::OptScope(const psml_options *o) : prev(t_opts) { if (o) t_opts = o; }
 OptScope::~OptScope() { t_opts = prev; }
@@ -306,7 +313,8 @@ psml_status psml_options_default(psml_options *out) {
 
 psml_status psml_ctx_set_options(psml_ctx ctx, const psml_options *o) {
     if (!ctx || !o) return fail(PSML_ERR_INVALID, "null argument");
-    if (o->seg_backend < 0 || o->seg_backend > 2 || o->msb_chain < 0 || o->msb_chain > 1 || o->deal_after < 0)
+    if (o->seg_backend < 0 || o->seg_backend > 2 || o->msb_chain < 0 || o->msb_chain > 1 || o->deal_after < 0 ||
+        o->deal_on_launch < 0 || o->deal_on_launch > 1)
         return fail(PSML_ERR_INVALID, "option out of range");
     reinterpret_cast<Ctx *>(ctx)->opts = *o;
     return PSML_OK;

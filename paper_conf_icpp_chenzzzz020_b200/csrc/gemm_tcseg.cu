@@ -522,13 +522,19 @@ psml_status tc_seg_group(const SegArgs<uint64_t> *jobs, int njobs, cudaStream_t 
     cfg.blockDim = dim3(NT);
     cfg.dynamicSmemBytes = SMEM_BYTES;
     cfg.stream = stream;
-    cudaLaunchAttribute attr[2];
+    cudaLaunchAttribute attr[3];
     attr[0].id = cudaLaunchAttributeClusterDimension;
     attr[0].val.clusterDim.x = 1; attr[0].val.clusterDim.y = 1; attr[0].val.clusterDim.z = (unsigned)ks;
     attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
     attr[1].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
     cfg.attrs = attr;
     cfg.numAttrs = 2;
+    if (cudaEvent_t ev = take_launch_event()) {   // fires once every CTA of this grid is resident
+        attr[2].id = cudaLaunchAttributeLaunchCompletionEvent;
+        attr[2].val.launchCompletionEvent.event = ev;
+        attr[2].val.launchCompletionEvent.flags = 0;
+        cfg.numAttrs = 3;
+    }
     ProfScope prof(PROF_TC, stream, work);
     PSML_CUDA_TRY(cudaLaunchKernelEx(&cfg, tcseg::tc_seg_kernel, g));
     g_launches.fetch_add(1, std::memory_order_relaxed);

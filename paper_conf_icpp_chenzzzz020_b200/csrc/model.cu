@@ -137,6 +137,8 @@ struct psml_model_s {
     int deal_pending_pool = -1;        // capture in progress: dealer branch not forked yet
     int deal_after = 0, deal_stage = 0;
     bool deal_alone = false;           // dealer being captured after the online chain (full PRG grid)
+    bool deal_on_launch = false;       // fork the dealer at the first product's launch completion
+    bool fork_event_armed = false;     // ev_late is that launch's completion event
     // split deployment capture (psml_party_capture_step): the party, its pair transport and its
     // data-parallel communicator; cap_party < 0 = the co-resident engine
     int cap_party = -1;
@@ -521,7 +523,7 @@ static psml_status build_plan(psml_model_s *m, int pool, bool infer_only) {
         switch (it.kind) {
         case IT_MATRIX:
         case IT_CONV_FWD:
-        case IT_CONV_GW:
+        case IT_CONV_GW: {
             job(PJ_PAIR, {TAG_U0, TAG_U1}, cid, it.U.n, {it.U.p[0], it.U.p[1]}, sr ? kp * it.U.n / 8 : 0);
             job(PJ_PAIR, {TAG_V0, TAG_V1}, cid, it.V.n, {it.V.p[0], it.V.p[1]}, 0);
             job(PJ_SINGLE, {TAG_Z0}, cid, it.Z.n, {it.Z.p[0]}, sr ? kp * it.Z.n / 8 : 0);
@@ -539,6 +541,7 @@ static psml_status build_plan(psml_model_s *m, int pool, bool infer_only) {
                 P.rest.push_back((int)k);
             }
             break;
+        }
         case IT_HAD: {
             const int64_t per = it.n / parts;
             for (int h = 0; h < parts; ++h) {
@@ -986,7 +989,11 @@ static psml_status deal_fork_point(psml_model_s *m, cudaStream_t s, bool force =
     if (!force && ++m->deal_stage < m->deal_after) return PSML_OK;
     const int pool = m->deal_pending_pool;
     m->deal_pending_pool = -1;
-    PSML_CUDA_TRY(cudaEventRecord(m->ev_late, s));
+    // ev_late = the fork edge: the completion of the online chain so far, or (deal_on_launch) the
+    // launch completion of the product just launched -- all its CTAs resident, so its SMs are
+    // taken before the dealer's grids arrive
+    if (!m->fork_event_armed) PSML_CUDA_TRY(cudaEventRecord(m->ev_late, s));
+    m->fork_event_armed = false;
     PSML_CUDA_TRY(cudaStreamWaitEvent(m->side, m->ev_late, 0));
     m->deal_alone = force;
     const psml_status st = deal_pool(m, pool, 0, false, m->side, deal_s2(m));
@@ -1080,7 +1087,13 @@ static psml_status fused_forward_backward(psml_model_s *m, const T *const X[2], 
     T *yo[2] = {m->yhat.p[0], m->yhat.p[1]};
     for (int l = 0; l < nl; ++l) {
         SegArgs<T> a = seg(l, OP_FWD, m->z[l].p[0], m->z[l].p[1], F);
+        const bool arm = l == 0 && m->deal_on_launch && m->deal_pending_pool >= 0;
+        if (arm) arm_launch_event(m->ev_late);
         PSML_TRY(launch_seg_group<T>(&a, 1, s, m->ctx->sm_count));
+        if (arm) {
+            m->fork_event_armed = take_launch_event() == nullptr;   // consumed by a tcgen05 launch
+            if (m->fork_event_armed) m->deal_stage = m->deal_after - 1;   // fork right here
+        }
         PSML_TRY(deal_fork_point(m, s));
         const int64_t w = m->dims[l + 1];
         if (l < nl - 1) {
@@ -1988,6 +2001,9 @@ static psml_status capture_one(psml_model_s *m, int pool, const T *const X[2], c
         // dealer forks at the start of the step (measured: 51.6K vs 49.4K samples/s forked after)
         m->deal_after = (fused_eligible(m) && m->cap_party < 0) ? after : 0;
         m->deal_stage = 0;
+        m->deal_on_launch = m->deal_after > 0 && cur_opts().deal_on_launch != 0;
+        if (m->deal_on_launch) m->deal_after = 2;   // the fork point right after the first product
+        m->fork_event_armed = false;
         if (st == PSML_OK && m->deal_after == 0) {
             st = deal_pool(m, 1 - pool, 0, false, m->side, deal_s2(m));
             if (st == PSML_OK) advance_word_kernel<<<1, 1, 0, m->side>>>(m->step_dev);

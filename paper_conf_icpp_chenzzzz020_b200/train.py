@@ -18,9 +18,18 @@ import torch
 from . import psml
 from .parallel import dp_update_shift, ring_allreduce_
 
+# The fixed seeds are the REPRODUCIBLE configuration (tests against the oracle, benchmarks): anyone
+# knowing them can regenerate every share and mask.  A deployment draws secret ones (fresh_seeds).
 DATA_SEED = 0x50534D4C
 SHARE_SEED = DATA_SEED + 1
 DEALER_SEED = DATA_SEED + 2
+
+
+def fresh_seeds():
+    """(share_seed, dealer_seed) from the OS CSPRNG, for a deployment: the client's sharing seed
+    and the dealer's seed are then secret (the ChaCha20 keys of DESIGN.md R1 / R23)."""
+    import secrets
+    return secrets.randbits(64), secrets.randbits(64)
 OP_SHARE = 7
 INIT_STEP = 0xFFFFFFFF
 KINDS = {"linreg": psml.LINREG, "logreg": psml.LOGREG, "mlp": psml.MLP, "cnn": psml.CNN, "svm": psml.SVM,
@@ -41,13 +50,14 @@ class SecureTrainer:
 
     def __init__(self, task, W_init, batch=128, pair_id=0, dims=None, backend=0,
                  frac_bits=13, master_frac_bits=27, lr_shift=14, compare="a2b", dealer_seed=DEALER_SEED,
-                 deal_role=0, w_shares=None, mask_reuse=False, strong_pairs=0):
+                 deal_role=0, w_shares=None, mask_reuse=False, strong_pairs=0, share_seed=SHARE_SEED):
         self.task = task
         self.ctx = psml.Ctx(l=64, frac_bits=frac_bits, backend=backend)
         self.ring = self.ctx.ring
         self.master_ring = psml.Ring(64, master_frac_bits)
         self.pair_id = pair_id
         self.batch = batch
+        self.share_seed = share_seed   # the client's sharing seed (secret in a deployment: fresh_seeds)
         # strong scaling (R28): strong_pairs pairs share one global batch of
         # strong_pairs * batch rows; this pair trains rows [pair_id * batch, (pair_id + 1) * batch)
         self.strong_pairs = strong_pairs
@@ -63,7 +73,7 @@ class SecureTrainer:
                 self.model.set_master(layer, w_shares[layer])
                 continue
             w = psml.encode(self.master_ring, torch.as_tensor(W, dtype=torch.float64))
-            Wm = psml.share(self.ring, SHARE_SEED, call_id(0, INIT_STEP, layer, OP_SHARE, 2), w)
+            Wm = psml.share(self.ring, self.share_seed, call_id(0, INIT_STEP, layer, OP_SHARE, 2), w)
             self.model.set_master(layer, Wm)
         self.out_dim = self.model.layer_shape(self.model.n_layers - 1)[1]
 
@@ -83,15 +93,15 @@ class SecureTrainer:
         cx = call_id(self.pair_id, step, 0, OP_SHARE, 0)
         cy = call_id(self.pair_id, step, 0, OP_SHARE, 1)
         if torch.is_tensor(X) and X.dtype == torch.uint8:
-            Xs = psml.encode_share_u8(self.ring, SHARE_SEED, cx, X if X.is_cuda else X.cuda(non_blocking=True),
+            Xs = psml.encode_share_u8(self.ring, self.share_seed, cx, X if X.is_cuda else X.cuda(non_blocking=True),
                                       255.0, out=outX)
         else:
-            Xs = psml.encode_share(self.ring, SHARE_SEED, cx, _dev64(X), out=outX)
+            Xs = psml.encode_share(self.ring, self.share_seed, cx, _dev64(X), out=outX)
         if torch.is_tensor(Y) and Y.dtype == torch.uint8:
-            Ys = psml.encode_share_onehot(self.ring, SHARE_SEED, cy, Y if Y.is_cuda else Y.cuda(non_blocking=True),
+            Ys = psml.encode_share_onehot(self.ring, self.share_seed, cy, Y if Y.is_cuda else Y.cuda(non_blocking=True),
                                           self.out_dim, out=outY)
         else:
-            Ys = psml.encode_share(self.ring, SHARE_SEED, cy, _dev64(Y), out=outY)
+            Ys = psml.encode_share(self.ring, self.share_seed, cy, _dev64(Y), out=outY)
         return Xs, Ys
 
     def share_batch(self, X, Y, step):
@@ -129,7 +139,7 @@ class SecureTrainer:
             self.model.deal(step)          # prime the pipeline (first step or a jump in step ids)
         if (torch.is_tensor(X) and torch.is_tensor(Y) and X.is_cuda and Y.is_cuda and X.dtype == torch.float64
                 and Y.dtype == torch.float64):
-            self.model.step_device(X.contiguous(), Y.contiguous(), SHARE_SEED, step)
+            self.model.step_device(X.contiguous(), Y.contiguous(), self.share_seed, step)
         else:
             self._client_share(X, Y, step, outX=self.Xbuf, outY=self.Ybuf)
             self.model.step_graph(step)
@@ -141,7 +151,7 @@ class SecureTrainer:
         uint64, 2 x batch x d_L) -- one library call (psml_model_step_host), asynchronous."""
         if self.pipelined and self._next_dealt != step:
             self.model.deal(step)
-        self.model.step_host(q, y, SHARE_SEED, step, yhat_host)
+        self.model.step_host(q, y, self.share_seed, step, yhat_host)
         self._next_dealt = step + 1
 
     def deal(self, step, infer_only=False):

@@ -278,3 +278,23 @@ def test_mask_reuse_bitexact_vs_oracle(T, task):
         torch.cuda.synchronize()
         _compare_shares(tr, om)
     tr.close()
+
+
+def test_fresh_secret_seeds_train_the_same_model(T):
+    """A deployment's secret seeds (train.fresh_seeds: OS CSPRNG share and dealer seeds) give other
+    shares and masks but the same decoded model (up to the SecureML truncation LSBs)."""
+    task = "mlp"
+    Wi = synth.init_weights(task)
+    share_seed, dealer_seed = T.fresh_seeds()
+    a = T.SecureTrainer(task, Wi)
+    b = T.SecureTrainer(task, Wi, share_seed=share_seed, dealer_seed=dealer_seed)
+    for s in range(3):
+        X, Y = synth.batch(task, s)
+        for tr in (a, b):
+            tr.step(torch.from_numpy(X), torch.from_numpy(Y), s)
+    torch.cuda.synchronize()
+    assert not np.array_equal(to_np(a.master_shares(0)[0]), to_np(b.master_shares(0)[0]))
+    for wa, wb in zip(a.master_weights(), b.master_weights()):
+        assert float((wa - wb).abs().max()) < 2.0 ** -14
+    a.close()
+    b.close()

@@ -37,8 +37,11 @@ prof.export_chrome_trace(out)
 ev = [e for e in json.load(open(out))["traceEvents"] if e.get("cat") == "kernel"]
 ev.sort(key=lambda e: e["ts"])
 # a step starts at each encode_share pair (client launches before each replay)
-starts = [e["ts"] for i, e in enumerate(ev) if "encode_share" in e["name"]
-          and (i == 0 or "encode_share" not in ev[i - 1]["name"])]
+def _share(e):   # the client's share launch(es) open each step
+    return "encode_share" in e["name"] or "client_share" in e["name"]
+
+
+starts = [e["ts"] for i, e in enumerate(ev) if _share(e) and (i == 0 or not _share(ev[i - 1]))]
 print(f"{len(ev)} kernels, {len(starts)} steps; mean step {(starts[-1] - starts[0]) / (len(starts) - 1):.1f} us")
 for k in range(len(starts) - 3, len(starts) - 1):
     t0, t1 = starts[k], starts[k + 1]
