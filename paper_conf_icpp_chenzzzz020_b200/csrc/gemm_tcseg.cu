@@ -26,6 +26,7 @@ namespace psml {
 namespace tcseg {
 
 constexpr int BM = 128, BN = 64, BK = 32, NT = 256, STAGES = 2, L = 8;
+constexpr int NTH = NT + 32;   // NT producer threads (loads, limb split, epilogue) + the MMA warp
 constexpr int A_TILE = BM * BK;                     // bytes per limb plane of one A block
 constexpr int B_TILE = BN * BK;                     // bytes per limb plane of one B block
 constexpr int STAGE_BYTES = L * (A_TILE + B_TILE);  // 48 KB of limb planes per K block
@@ -37,7 +38,7 @@ constexpr int RAW_STAGE_BYTES = RAW_A_BYTES + RAW_B_BYTES;
 constexpr int RAW_OFF = STAGES * STAGE_BYTES;
 constexpr int PIPE_BYTES = RAW_OFF + RAW_STAGES * RAW_STAGE_BYTES;
 static_assert(BM * RED_PITCH * 8 <= PIPE_BYTES, "reduction tile must fit the pipeline region");
-constexpr size_t SMEM_BYTES = PIPE_BYTES + 8 * (STAGES + 2) + 16;   // > 114 KB: one CTA per SM
+constexpr size_t SMEM_BYTES = PIPE_BYTES + 8 * (2 * STAGES + 2) + 16;   // > 114 KB: one CTA per SM
 constexpr int MAX_KS = 16;
 
 struct Group {
@@ -46,7 +47,6 @@ struct Group {
     int tiles_n[SEG_MAX_JOBS], tiles_m[SEG_MAX_JOBS];
     int kb_per_split[SEG_MAX_JOBS];
     int njobs, ks;
-    int debug_mmas;   // TCSEG_TIMING builds: issue only limb pairs with 8 p + q < debug_mmas
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -108,8 +108,10 @@ __device__ __forceinline__ uint64_t sdesc(uint32_t addr) {
     return (uint64_t)((addr >> 4) & 0x3FFFu) | ((uint64_t)(128 >> 4) << 16) | ((uint64_t)(256 >> 4) << 32) |
            (1ull << 46);
 }
-// kind::i8 instruction descriptor: D s32, A/B u8, both K-major, M = 128, N = BN.
-constexpr uint32_t IDESC = (2u << 4) | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
+// kind::i8 instruction descriptor: D s32, A/B u8, both K-major, M = BM, N = n (a multiple of 16, <= 256).
+__device__ __forceinline__ uint32_t idesc_i8(int n) {
+    return (2u << 4) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
+}
 
 // 4 x 4 byte transpose: w[i] = bytes (b0..b3) of word i -> o[p] = (w0.bp, w1.bp, w2.bp, w3.bp)
 __device__ __forceinline__ void bt4(uint32_t w0, uint32_t w1, uint32_t w2, uint32_t w3, uint32_t o[4]) {
@@ -159,12 +161,48 @@ __device__ __forceinline__ void slice_store(const SegArgs<uint64_t> &a, int p, i
     }
 }
 
-// grid (total tiles, 1, ks), cluster (1, 1, ks), 256 threads, SMEM_BYTES dynamic shared memory.
-__global__ void __launch_bounds__(NT, 1) tc_seg_kernel(const __grid_constant__ Group g) {
+// The same epilogue, summing the slice's rows straight out of every cluster CTA's partial tile
+// (ld.shared::cluster: distributed shared memory reads, KS loads per element in flight).
+template <int KS>
+__device__ __forceinline__ void slice_sum_store(const SegArgs<uint64_t> &a, int p, int64_t m0, int64_t n0, int rank,
+                                                uint32_t red_u32, const uint64_t zpre[ZPF]) {
+    constexpr int PER = BM * BN / KS, NEL = PER / NT;
+    const int tid = threadIdx.x, party = a.party[p];
+    uint32_t peer[KS];
+#pragma unroll
+    for (int q = 0; q < KS; ++q) asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(peer[q]) : "r"(red_u32), "r"(q));
+#pragma unroll
+    for (int i = 0; i < NEL; ++i) {
+        const int e = rank * PER + tid + NT * i;
+        const int r = e / BN, c = e % BN;
+        const uint32_t off = (uint32_t)(r * RED_PITCH + c) * 8;
+        uint64_t part[KS];
+#pragma unroll
+        for (int q = 0; q < KS; ++q) asm volatile("ld.shared::cluster.u64 %0, [%1];" : "=l"(part[q]) : "r"(peer[q] + off));
+        uint64_t sum = 0;
+#pragma unroll
+        for (int q = 0; q < KS; ++q) sum += part[q];
+        const int64_t m = m0 + r, n = n0 + c;
+        const int64_t o = (m < a.M ? m : a.M - 1) * a.N + (n < a.N ? n : a.N - 1);
+        const uint64_t z = NEL <= ZPF ? zpre[i < ZPF ? i : 0] : ldg(a.Z[p] + o);
+        if (m < a.M && n < a.N) a.C[p][o] = trunc_share<uint64_t>(sum + z, party, a.trunc);
+    }
+}
+
+#ifndef PSML_TCSEG_RED
+#define PSML_TCSEG_RED 1   // split-K reduction: 0 bulk-copy .add.u64 into the owner CTA, 1 DSMEM reads
+#endif
+
+// grid (total tiles, 1, ks), cluster (1, 1, ks), NTH threads, SMEM_BYTES dynamic shared memory.
+// Warps 0-7 land the raw operand words (cp.async) and split them into limb planes; warp 8 issues
+// the MMAs of each limb stage as soon as its `full` barrier completes, so the tensor core works
+// on block i while the producers split block i + 1.
+__global__ void __launch_bounds__(NTH, 1) tc_seg_kernel(const __grid_constant__ Group g) {
     namespace cg = cooperative_groups;
     extern __shared__ __align__(1024) uint8_t smem[];
-    uint64_t *empty = (uint64_t *)(smem + PIPE_BYTES);
-    uint64_t *accum = empty + STAGES;
+    uint64_t *empty = (uint64_t *)(smem + PIPE_BYTES);   // limb stage free (MMAs of its block done)
+    uint64_t *full = empty + STAGES;                      // limb stage written by all NT producers
+    uint64_t *accum = full + STAGES;
     uint64_t *rbar = accum + 1;   // split-K reduction: peers' partial slices landed
     uint32_t *tmem_slot = (uint32_t *)(rbar + 1);
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -195,7 +233,10 @@ __global__ void __launch_bounds__(NT, 1) tc_seg_kernel(const __grid_constant__ G
     const uint64_t *Xp = a.X[p], *Ep = a.E, *Fp = a.F, *Vp = a.V[p];
 
     if (tid == 0) {
-        for (int s = 0; s < STAGES; ++s) mbar_init(smem_u32(&empty[s]), 1);
+        for (int s = 0; s < STAGES; ++s) {
+            mbar_init(smem_u32(&empty[s]), 1);
+            mbar_init(smem_u32(&full[s]), NT);
+        }
         mbar_init(smem_u32(accum), 1);
         mbar_init(smem_u32(rbar), 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -217,7 +258,7 @@ __global__ void __launch_bounds__(NT, 1) tc_seg_kernel(const __grid_constant__ G
 #pragma unroll
         for (int i = 0; i < ZPF; ++i) {
             zpre[i] = 0;
-            if (nel <= ZPF && i < nel) {
+            if (nel <= ZPF && i < nel && tid < NT) {
                 const int e = (int)blockIdx.z * (nel * NT) + tid + NT * i;
                 const int64_t m = m0 + e / BN, n = n0 + e % BN;
                 zpre[i] = ldg(a.Z[p] + (m < M ? m : M - 1) * N + (n < N ? n : N - 1));
@@ -311,58 +352,49 @@ __global__ void __launch_bounds__(NT, 1) tc_seg_kernel(const __grid_constant__ G
     // operands X_p / E / F it produces are read only after this wait.
     pdl_trigger();
     pdl_wait();
-    if (nblk > 0) issue(kb0, 0);
-    cp_async_commit();
-    if (nblk > 1) issue(kb0 + 1, 1);
-    cp_async_commit();
-    TS(2);
-    for (int i = 0; i < nblk; ++i) {
-        const int st = i % STAGES, rs = i % RAW_STAGES;
-#ifdef TCSEG_TIMING
-        uint64_t tq0, tq1, tq2, tq3, tq4;
-        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tq0));
-#endif
-        cp_async_wait1();   // this thread's chunks of block i have landed
-        __syncthreads();    // ... and every thread's
-#ifdef TCSEG_TIMING
-        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tq1));
-#endif
-        if (i >= STAGES) mbar_wait(smem_u32(&empty[st]), (uint32_t)((i / STAGES - 1) & 1));
-#ifdef TCSEG_TIMING
-        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tq2));
-#endif
-        stash(rs, st);
-#ifdef TCSEG_TIMING
-        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tq3));
-#endif
-        __syncthreads();    // limb stage st complete; raw stage rs free
-#ifdef TCSEG_TIMING
-        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(tq4));
-        if (tid == 0 && blockIdx.x == 0 && blockIdx.z == 0 && gridDim.x == 4)
-            printf("  blk i=%d: wait_data %llu wait_empty %llu stash %llu sync %llu\n", i, tq1 - tq0, tq2 - tq1,
-                   tq3 - tq2, tq4 - tq3);
-#endif
-        if (tid == 0) {
+    if (warp < NT / 32) {   // producers
+        if (nblk > 0) issue(kb0, 0);
+        cp_async_commit();
+        if (nblk > 1) issue(kb0 + 1, 1);
+        cp_async_commit();
+        TS(2);
+        for (int i = 0; i < nblk; ++i) {
+            const int st = i % STAGES, rs = i % RAW_STAGES;
+            cp_async_wait1();                                 // this thread's chunks of block i landed
+            asm volatile("bar.sync 1, %0;" ::"n"(NT) : "memory");   // ... and every producer's
+            if (i >= STAGES) mbar_wait(smem_u32(&empty[st]), (uint32_t)((i / STAGES - 1) & 1));
+            stash(rs, st);                                    // ends with fence.proxy.async
+            asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&full[st])) : "memory");
+            asm volatile("bar.sync 1, %0;" ::"n"(NT) : "memory");   // raw stage rs read by everyone
+            if (i + 2 < nblk) issue(kb0 + i + 2, rs);
+            cp_async_commit();
+        }
+    } else if (lane == 0) {   // the MMA warp: 36 limb-pair MMAs per stage into the shift accumulators
+        for (int i = 0; i < nblk; ++i) {
+            const int st = i % STAGES;
+            mbar_wait(smem_u32(&full[st]), (uint32_t)((i / STAGES) & 1));
             fence_after();
             const uint32_t sa = smem_u32(smem + st * STAGE_BYTES), sb = sa + L * A_TILE;
+            // A limb pa times B limbs 0 .. 7 - pa: the B planes lie back to back in the canonical
+            // layout (plane stride = 8 row groups x SBO), so they form ONE N = 64 (8 - pa) operand
+            // whose product lands in TMEM columns (pa + q) 64 = shift accumulators S_pa .. S_7 --
+            // 12 MMAs of N <= 256 per K block instead of 36 of N = 64, A read from shared memory
+            // 12 times instead of 36
 #pragma unroll
             for (int pa = 0; pa < L; ++pa) {
                 const uint64_t ad = sdesc(sa + pa * A_TILE);
 #pragma unroll
-                for (int qb = 0; qb < L - pa; ++qb) {
-#ifdef TCSEG_TIMING
-                    if (g.debug_mmas && pa * 8 + qb >= g.debug_mmas) continue;   // timing experiments only
-#endif
-                    mma_i8(tmem + (uint32_t)((pa + qb) * BN), ad, sdesc(sb + qb * B_TILE), IDESC,
+                for (int q0 = 0; q0 < L - pa; q0 += 4) {
+                    const int nq = (L - pa - q0) < 4 ? (L - pa - q0) : 4;
+                    mma_i8(tmem + (uint32_t)((pa + q0) * BN), ad, sdesc(sb + q0 * B_TILE), idesc_i8(nq * BN),
                            (i > 0 || pa > 0) ? 1u : 0u);
                 }
             }
             commit(smem_u32(&empty[st]));
         }
-        if (i + 2 < nblk) issue(kb0 + i + 2, rs);
-        cp_async_commit();
+        commit(smem_u32(accum));
     }
-    if (tid == 0) commit(smem_u32(accum));
+    __syncwarp();
     TS(3);
 
     // ---- partial tile: sum_s S_s 2^{8s} (u64, exact) -> reduction buffer ----
@@ -370,11 +402,11 @@ __global__ void __launch_bounds__(NT, 1) tc_seg_kernel(const __grid_constant__ G
     mbar_wait(smem_u32(accum), 0);
     TS(4);
     fence_after();
-    if (warp < 4) {
-        const int row = warp * 32 + lane;
-        const uint32_t lane_base = tmem + ((uint32_t)(warp * 32) << 16);
+    if (warp < NT / 32) {   // warps w and w + 4 share TMEM lanes 32 (w % 4) ..; each drains half the columns
+        const int row = (warp & 3) * 32 + lane;
+        const uint32_t lane_base = tmem + ((uint32_t)((warp & 3) * 32) << 16);
 #pragma unroll 1
-        for (int j0 = 0; j0 < BN; j0 += 16) {
+        for (int j0 = (warp >> 2) * (BN / 2); j0 < (warp >> 2) * (BN / 2) + BN / 2; j0 += 16) {
             uint64_t acc[16];
 #pragma unroll
             for (int j = 0; j < 16; ++j) acc[j] = 0;
@@ -398,39 +430,51 @@ __global__ void __launch_bounds__(NT, 1) tc_seg_kernel(const __grid_constant__ G
     // tile (R = BM / ks) are added (cp.reduce.async.bulk .add.u64) into CTA q's copy; CTA q then
     // runs the epilogue on its fully reduced slice from local shared memory ----
     const int ks = g.ks;
-    const uint32_t slice_bytes = (uint32_t)(BM / ks) * RED_PITCH * 8;
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // red writes -> bulk-copy proxy
-    if (tid == 0 && ks > 1)
-        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(rbar)),
-                     "r"((uint32_t)(ks - 1) * slice_bytes)
-                     : "memory");
-    fence_before();
     cg::cluster_group cluster = cg::this_cluster();
-    cluster.sync();   // every partial written, every receiver armed, every pipeline idle
-    TS(6);
     const int rank = (int)cluster.block_rank();
-    if (tid == 0 && ks > 1) {
-        const uint32_t base = smem_u32(red), bar = smem_u32(rbar);
-        for (int q = 0; q < ks; ++q) {
-            if (q == rank) continue;
-            const uint32_t src = base + (uint32_t)q * slice_bytes;
-            uint32_t dst, dbar;
-            asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(dst) : "r"(src), "r"(q));
-            asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(dbar) : "r"(bar), "r"(q));
-            asm volatile(
-                "cp.reduce.async.bulk.shared::cluster.shared::cta.mbarrier::complete_tx::bytes.add.u64 [%0], [%1], "
-                "%2, [%3];" ::"r"(dst),
-                "r"(src), "r"(slice_bytes), "r"(dbar)
-                : "memory");
+    if (PSML_TCSEG_RED == 1 && ks > 1) {
+        cluster.sync();   // every CTA's partial tile written
+        TS(6);
+        const uint32_t rb = smem_u32(red);
+        if (tid < NT) switch (ks) {
+        case 2: slice_sum_store<2>(a, p, m0, n0, rank, rb, zpre); break;
+        case 4: slice_sum_store<4>(a, p, m0, n0, rank, rb, zpre); break;
+        case 8: slice_sum_store<8>(a, p, m0, n0, rank, rb, zpre); break;
+        default: slice_sum_store<16>(a, p, m0, n0, rank, rb, zpre); break;
         }
-    }
-    if (ks > 1) mbar_wait(smem_u32(rbar), 0);
-    switch (ks) {
-    case 1: slice_store<1>(a, p, m0, n0, rank, red, zpre); break;
-    case 2: slice_store<2>(a, p, m0, n0, rank, red, zpre); break;
-    case 4: slice_store<4>(a, p, m0, n0, rank, red, zpre); break;
-    case 8: slice_store<8>(a, p, m0, n0, rank, red, zpre); break;
-    default: slice_store<16>(a, p, m0, n0, rank, red, zpre); break;
+    } else {
+        const uint32_t slice_bytes = (uint32_t)(BM / ks) * RED_PITCH * 8;
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // red writes -> bulk-copy proxy
+        if (tid == 0 && ks > 1)
+            asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(rbar)),
+                         "r"((uint32_t)(ks - 1) * slice_bytes)
+                         : "memory");
+        fence_before();
+        cluster.sync();   // every partial written, every receiver armed, every pipeline idle
+        TS(6);
+        if (tid == 0 && ks > 1) {
+            const uint32_t base = smem_u32(red), bar = smem_u32(rbar);
+            for (int q = 0; q < ks; ++q) {
+                if (q == rank) continue;
+                const uint32_t src = base + (uint32_t)q * slice_bytes;
+                uint32_t dst, dbar;
+                asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(dst) : "r"(src), "r"(q));
+                asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(dbar) : "r"(bar), "r"(q));
+                asm volatile(
+                    "cp.reduce.async.bulk.shared::cluster.shared::cta.mbarrier::complete_tx::bytes.add.u64 [%0], [%1], "
+                    "%2, [%3];" ::"r"(dst),
+                    "r"(src), "r"(slice_bytes), "r"(dbar)
+                    : "memory");
+            }
+        }
+        if (ks > 1) mbar_wait(smem_u32(rbar), 0);
+        if (tid < NT) switch (ks) {
+        case 1: slice_store<1>(a, p, m0, n0, rank, red, zpre); break;
+        case 2: slice_store<2>(a, p, m0, n0, rank, red, zpre); break;
+        case 4: slice_store<4>(a, p, m0, n0, rank, red, zpre); break;
+        case 8: slice_store<8>(a, p, m0, n0, rank, red, zpre); break;
+        default: slice_store<16>(a, p, m0, n0, rank, red, zpre); break;
+        }
     }
     cluster.sync();   // peers' shared memory stays alive until every CTA has read it
     TS(7);
@@ -474,7 +518,7 @@ psml_status tc_seg_group(const SegArgs<uint64_t> *jobs, int njobs, cudaStream_t 
         if (cudaFuncSetAttribute(tc_seg_kernel, cudaFuncAttributeNonPortableClusterSizeAllowed, 1) == cudaSuccess) {
             cudaLaunchConfig_t q = {};
             q.gridDim = dim3(MAX_KS, 1, MAX_KS);
-            q.blockDim = dim3(NT);
+            q.blockDim = dim3(NTH);
             q.dynamicSmemBytes = SMEM_BYTES;
             cudaLaunchAttribute at[1];
             at[0].id = cudaLaunchAttributeClusterDimension;
@@ -504,9 +548,6 @@ psml_status tc_seg_group(const SegArgs<uint64_t> *jobs, int njobs, cudaStream_t 
     }
     g.tile_begin[njobs] = tiles;
     g.njobs = njobs;
-#ifdef TCSEG_TIMING
-    if (const char *e = getenv("PSML_TCSEG_MMAS")) g.debug_mmas = atoi(e);
-#endif
     // K split: double ks while the grid stays within 1/PSML_TCSEG_FILL of the SMs (default 2: the
     // rest stays with the dealer branch) and each split keeps >= 2 K blocks
     const int fill = PSML_TCSEG_FILL;
@@ -519,7 +560,7 @@ psml_status tc_seg_group(const SegArgs<uint64_t> *jobs, int njobs, cudaStream_t 
     }
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)tiles, 1, (unsigned)ks);
-    cfg.blockDim = dim3(NT);
+    cfg.blockDim = dim3(NTH);
     cfg.dynamicSmemBytes = SMEM_BYTES;
     cfg.stream = stream;
     cudaLaunchAttribute attr[3];
