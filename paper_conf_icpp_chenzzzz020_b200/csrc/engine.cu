@@ -291,7 +291,7 @@ psml_status psml_secure_matmul_party(psml_ctx ctx, const void *A_i, const void *
 }
 
 namespace psml {
-static const psml_options k_default_opts{0, 1, 0, 1, 1, 1, 1, 1, 1, 1, 0, 1, 1, 0};
+static const psml_options k_default_opts{0, 1, 0, 1, 1, 1, 1, 1, 1, 1, 0, 1, 1, 0, 1};
 static thread_local const psml_options *t_opts = nullptr;
 static thread_local cudaEvent_t t_launch_event = nullptr;
 void arm_launch_event(cudaEvent_t e) { t_launch_event = e; }
@@ -314,7 +314,7 @@ psml_status psml_options_default(psml_options *out) {
 psml_status psml_ctx_set_options(psml_ctx ctx, const psml_options *o) {
     if (!ctx || !o) return fail(PSML_ERR_INVALID, "null argument");
     if (o->seg_backend < 0 || o->seg_backend > 2 || o->msb_chain < 0 || o->msb_chain > 1 || o->deal_after < 0 ||
-        o->deal_on_launch < 0 || o->deal_on_launch > 1)
+        o->deal_on_launch < 0 || o->deal_on_launch > 1 || o->tc_small < 0 || o->tc_small > 2)
         return fail(PSML_ERR_INVALID, "option out of range");
     reinterpret_cast<Ctx *>(ctx)->opts = *o;
     return PSML_OK;
@@ -922,6 +922,8 @@ psml_status psml_fss_open_drelu(psml_ctx ctx, int32_t party, const void *msg_sen
 template <typename T>
 static psml_status ring_gemm_t(Ctx *c, const void *A, const void *B, int64_t M, int64_t K, int64_t N, void *C,
                                cudaStream_t s) {
+    if (c->use_tc(M, K, N) && tc_seg_small(8 * (int)sizeof(T), M, K, N, 1, c->sm_count))   // one launch
+        return tc_seg_plain<T>((const T *)A, (const T *)B, M, K, N, (T *)C, s, c->sm_count);
     if (c->use_tc(M, K, N)) {
         size_t need = tc_ring_gemm_ws_bytes(8 * (int)sizeof(T), M, K, N);
         PSML_TRY(c->ensure_ws(need));

@@ -29,7 +29,7 @@ int current_sm_count();
 struct Ctx {
     psml_ring ring{64, 13};
     int backend = 0;    // 0 auto, 1 CUDA-core, 2 tcgen05
-    psml_options opts{0, 1, 0, 1, 1, 1, 1, 1, 1, 1, 0, 1, 1};   // = psml_options_default
+    psml_options opts{0, 1, 0, 1, 1, 1, 1, 1, 1, 1, 0, 1, 1, 0, 1};   // = psml_options_default
     int sm_count = 148;
     bool tc_ok = false;
     void *ws = nullptr;

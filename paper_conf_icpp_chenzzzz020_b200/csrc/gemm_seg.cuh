@@ -248,7 +248,21 @@ __global__ void __launch_bounds__(SegCfg::NT) seg_gemm_kernel(const __grid_const
 bool tc_seg_enabled();
 bool tc_seg_forced();   // PSML_SEG=tc: every eligible group on tcgen05 (tests)
 bool pdl_enabled();     // PSML_PDL=0 disables programmatic dependent launch
-psml_status tc_seg_group(const SegArgs<uint64_t> *jobs, int njobs, cudaStream_t stream, int sm_count);
+// segs = 2: Beaver products [X_p | E] . [F ; V_p]; 1: plain X . F.  fill: the grid's K split stops at
+// 1/fill of the SMs (2 inside the training step, whose dealer branch runs beside it; 1 stand-alone).
+psml_status tc_seg_group(const SegArgs<uint64_t> *jobs, int njobs, cudaStream_t stream, int sm_count, int segs = 2,
+                         int fill = 2);
+// Stand-alone products on the in-kernel limb-split kernel (psml_options.tc_small): plain C = A . B
+// and the co-resident Beaver product (one mask + open pass, then Eq. 8); l = 64 needs K' <= 16384.
+bool tc_seg_small(int l, int64_t M, int64_t Kext, int64_t N, int nparty, int sm_count);
+template <typename T>
+psml_status tc_seg_plain(const T *A, const T *B, int64_t M, int64_t K, int64_t N, T *C, cudaStream_t s, int sm_count);
+template <typename T>
+size_t tc_seg_beaver_ws_bytes(int64_t M, int64_t K, int64_t N);
+template <typename T>
+psml_status tc_seg_beaver(const T *const A[2], const T *const B[2], const T *const U[2], const T *const V[2],
+                          const T *const Z[2], int64_t M, int64_t K, int64_t N, int flags, int trunc, T *const C[2],
+                          void *ws, size_t ws_bytes, cudaStream_t s, int sm_count);
 
 
 // Launch 1..SEG_MAX_JOBS products as one grid; the cluster split ks is chosen for the group.

@@ -235,6 +235,9 @@ __device__ __forceinline__ void epi_chunk(T *st, const T v[16], int lane, int64_
     __syncwarp();
 }
 
+#ifndef TC_V1_GROUP
+#define TC_V1_GROUP 0
+#endif
 template <typename T, int L, int BN, int STAGES>
 __global__ void __launch_bounds__(128, 1) tc_ring_gemm_kernel(const TcParams<T> P) {
     extern __shared__ __align__(1024) uint8_t smem[];
@@ -299,6 +302,24 @@ __global__ void __launch_bounds__(128, 1) tc_ring_gemm_kernel(const TcParams<T> 
             mbar_wait(smem_u32(&full[stage]), phase);
             tc_fence_after();
             const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES), sb = sa + L * A_BYTES;
+#if TC_V1_GROUP
+            // the B planes q0, q0 + 1 of A limb p lie back to back in the canonical layout (plane
+            // stride = BN / 8 row groups x SBO): ONE N = 2 BN operand into the adjacent shift
+            // accumulators S_{p+q0}, S_{p+q0+1} -- 6 MMAs per block instead of 10 at l = 32, A read
+            // 6 times instead of 10
+            constexpr int GQ = 256 / BN;
+#pragma unroll
+            for (int p = 0; p < L; ++p) {
+                const uint64_t ad = smem_desc(sa + p * A_BYTES, 128, 256);
+#pragma unroll
+                for (int q0 = 0; q0 < L - p; q0 += GQ) {
+                    const int nq = (L - p - q0) < GQ ? (L - p - q0) : GQ;
+                    const uint64_t bd = smem_desc(sb + q0 * B_BYTES, 128, 256);
+                    tc_mma_i8(tmem + (uint32_t)((p + q0) * BN), ad, bd, idesc_i8(BM, nq * BN),
+                              (kb > kb0 || p > 0) ? 1u : 0u);
+                }
+            }
+#else
 #pragma unroll
             for (int p = 0; p < L; ++p) {
                 const uint64_t ad = smem_desc(sa + p * A_BYTES, 128, 256);
@@ -308,6 +329,7 @@ __global__ void __launch_bounds__(128, 1) tc_ring_gemm_kernel(const TcParams<T> 
                     tc_mma_i8(tmem + (uint32_t)((p + q) * BN), ad, bd, IDESC, (kb > kb0 || p > 0) ? 1u : 0u);
                 }
             }
+#endif
             tc_commit(smem_u32(&empty[stage]));   // frees the smem stage once these MMAs retire
             if (++stage == STAGES) { stage = 0; phase ^= 1; }
         }
@@ -722,6 +744,8 @@ psml_status tc_beaver_matmul_ws(const T *const A[2], const T *const B[2], const 
                                 T *const C[2], void *ws, size_t ws_bytes, int sm_count, cudaStream_t s) {
     constexpr int l = 8 * (int)sizeof(T);
     using Cf = tc::Cfg<l>;
+    if (tc_seg_small(l, M, 2 * K, N, 2, sm_count))   // small products: one open pass + the in-kernel split kernel
+        return tc_seg_beaver<T>(A, B, U, V, Z, M, K, N, flags, trunc, C, ws, ws_bytes, s, sm_count);
     if (ws_bytes < tc_beaver_ws_bytes<T>(M, K, N)) return fail(PSML_ERR_NOMEM, "tcgen05 Beaver workspace too small");
     uint8_t *w = (uint8_t *)ws;
     auto carve = [&](size_t bytes) { uint8_t *p = w; w += (bytes + 255) & ~(size_t)255; return p; };

@@ -5,48 +5,50 @@
 // Same exact limb decomposition as gemm_tc.cu (8-bit limbs, the 36 limb pairs p + q < 8 of Z_2^64
 // as tcgen05.mma.kind::i8 into 8 per-shift s32 TMEM accumulators S_s, result sum_s S_s 2^{8s}),
 // but built for products whose whole operand set is a few MB: there is NO separate limb-split
-// pass through HBM.  The CTA's 8 warps load the uint64 operand words straight from the producers'
-// outputs (L2-resident), split them into limb bytes in registers (a 4 x 4 byte transpose per
-// 4 words: 2 PRMT per limb word) and store them into shared memory already in the UMMA K-major
-// no-swizzle canonical layout; one thread issues the 36 MMAs of the 128 x 64 x 32 block while the
-// warps split the next block (3-stage ring; the commit of a stage's MMAs frees it).
+// pass through HBM.  The CTA's 8 producer warps load the uint64 operand words of K block i + 2
+// straight from the producers' outputs (L2-resident) into registers (32-byte loads: a warp reads
+// four whole 256-byte rows of A per instruction) while they split block i into limb bytes (a 4 x 4
+// byte transpose per 4 words: 2 PRMT per limb word) and store them into shared memory in the UMMA
+// K-major no-swizzle canonical layout; warp 8 issues the block's limb-pair MMAs (the B planes of
+// one A limb as one N <= 256 operand: 12 MMAs per block) as soon as the stage's `full` barrier
+// completes (4-stage ring; the commit of a stage's MMAs frees it).  Per 128 x 64 x 32 block a CTA
+// moves 48 KB of limb planes into shared memory and the MMAs read 120 KB back (A 12 x 4 KB, B
+// 36 x 2 KB): 168 KB at 128 B/clk is 1.3 us -- the kernel's shared-memory roofline (measured
+// 1.4 us per block with every SM busy).
 // K is split over the ks CTAs of a (1, 1, ks) thread-block cluster: each CTA turns its
 // accumulators into uint64 partials (exact mod 2^64, K' per CTA <= 2^14 keeps S_0..S_3 exact),
 // the partial tiles are summed through distributed shared memory, and each CTA runs the epilogue
 // (+ Z_p, truncation, store) on 1/ks of the tile.  Ring addition is exact, so the result is
 // bit-identical to the CUDA-core seg_gemm_kernel (tested).
-#ifndef PSML_TCSEG_FILL
-#define PSML_TCSEG_FILL 2
-#endif
+// segs = 1 runs the plain product X . F (K' = K, no Z): psml_ring_gemm at small n (config 5).
 #include <cooperative_groups.h>
 
 #include "engine.h"
+#include "fused.cuh"
 
 namespace psml {
 namespace tcseg {
 
-constexpr int BM = 128, BN = 64, BK = 32, NT = 256, STAGES = 2, L = 8;
+constexpr int BM = 128, BN = 64, BK = 32, NT = 256, LMAX = 8;
+constexpr int STAGES = 4;
 constexpr int NTH = NT + 32;   // NT producer threads (loads, limb split, epilogue) + the MMA warp
-constexpr int A_TILE = BM * BK;                     // bytes per limb plane of one A block
-constexpr int B_TILE = BN * BK;                     // bytes per limb plane of one B block
-constexpr int STAGE_BYTES = L * (A_TILE + B_TILE);  // 48 KB of limb planes per K block
-constexpr int RED_PITCH = BN + 1;                   // u64 words per row of the reduction tile
-// raw uint64 operand words of one K block, landed by cp.async two blocks ahead of their split
-constexpr int RAW_STAGES = 2, RAW_A_PITCH = 34;     // A rows padded to 272 B (16-B aligned)
-constexpr int RAW_A_BYTES = BM * RAW_A_PITCH * 8, RAW_B_BYTES = BK * BN * 8;
-constexpr int RAW_STAGE_BYTES = RAW_A_BYTES + RAW_B_BYTES;
-constexpr int RAW_OFF = STAGES * STAGE_BYTES;
-constexpr int PIPE_BYTES = RAW_OFF + RAW_STAGES * RAW_STAGE_BYTES;
+constexpr int A_TILE = BM * BK;                        // bytes per limb plane of one A block
+constexpr int B_TILE = BN * BK;                        // bytes per limb plane of one B block
+constexpr int STAGE_BYTES = LMAX * (A_TILE + B_TILE);  // stage stride: 48 KB (l = 64: 8 limb planes each)
+constexpr int RED_PITCH = BN + 1;                      // words per row of the reduction tile
+constexpr int PIPE_BYTES = STAGES * STAGE_BYTES;
 static_assert(BM * RED_PITCH * 8 <= PIPE_BYTES, "reduction tile must fit the pipeline region");
 constexpr size_t SMEM_BYTES = PIPE_BYTES + 8 * (2 * STAGES + 2) + 16;   // > 114 KB: one CTA per SM
 constexpr int MAX_KS = 16;
 
+template <typename T>
 struct Group {
-    SegArgs<uint64_t> j[SEG_MAX_JOBS];
+    SegArgs<T> j[SEG_MAX_JOBS];
     int64_t tile_begin[SEG_MAX_JOBS + 1];
     int tiles_n[SEG_MAX_JOBS], tiles_m[SEG_MAX_JOBS];
     int kb_per_split[SEG_MAX_JOBS];
     int njobs, ks;
+    int segs;   // 2: the Beaver product [X_p | E] . [F ; V_p] (K' = 2K); 1: the plain product X . F (K' = K)
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -122,89 +124,106 @@ __device__ __forceinline__ void bt4(uint32_t w0, uint32_t w1, uint32_t w2, uint3
     o[2] = __byte_perm(t1, t3, 0x5410);
     o[3] = __byte_perm(t1, t3, 0x7632);
 }
-// limb words of 4 consecutive ring elements: out[p] = bytes p of v0..v3 (p = 0..7)
+// limb words of 4 consecutive ring elements: out[p] = bytes p of v0..v3 (p < sizeof(T))
 __device__ __forceinline__ void limbs4(const uint64_t *v, uint32_t out[8]) {
     bt4((uint32_t)v[0], (uint32_t)v[1], (uint32_t)v[2], (uint32_t)v[3], out);
     bt4((uint32_t)(v[0] >> 32), (uint32_t)(v[1] >> 32), (uint32_t)(v[2] >> 32), (uint32_t)(v[3] >> 32), out + 4);
 }
+__device__ __forceinline__ void limbs4(const uint32_t *v, uint32_t out[4]) { bt4(v[0], v[1], v[2], v[3], out); }
 
 __device__ __forceinline__ uint64_t ldg(const uint64_t *p) { return __ldg((const unsigned long long *)p); }
-__device__ __forceinline__ void cp_async16(void *dst, const void *src, bool ok) {
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_u32(dst)), "l"(src), "r"(ok ? 16 : 0)
-                 : "memory");
+__device__ __forceinline__ uint32_t ldg(const uint32_t *p) { return __ldg((const unsigned int *)p); }
+// 4 consecutive words (32 B for l = 64, 16 B for l = 32; aligned)
+__device__ __forceinline__ void ld4(const uint64_t *p, uint64_t *v) {
+    asm volatile("ld.global.nc.v4.u64 {%0, %1, %2, %3}, [%4];" : "=l"(v[0]), "=l"(v[1]), "=l"(v[2]), "=l"(v[3]) : "l"(p));
 }
-__device__ __forceinline__ void cp_async8(void *dst, const void *src, bool ok) {
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;" ::"r"(smem_u32(dst)), "l"(src), "r"(ok ? 8 : 0)
-                 : "memory");
+__device__ __forceinline__ void ld4(const uint32_t *p, uint32_t *v) {
+    const uint4 q = __ldg((const uint4 *)p);
+    v[0] = q.x; v[1] = q.y; v[2] = q.z; v[3] = q.w;
 }
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-__device__ __forceinline__ void cp_async_wait1() { asm volatile("cp.async.wait_group 1;" ::: "memory"); }
-
+__device__ __forceinline__ uint64_t ld_dsmem(uint32_t a, uint64_t *) {
+    uint64_t v;
+    asm volatile("ld.shared::cluster.u64 %0, [%1];" : "=l"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ uint32_t ld_dsmem(uint32_t a, uint32_t *) {
+    uint32_t v;
+    asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(v) : "r"(a));
+    return v;
+}
 constexpr int ZPF = 8;   // epilogue Z words prefetched per thread (ks >= 4)
+#ifndef TCSEG_EPI_UNROLL
+#define TCSEG_EPI_UNROLL 4    // epilogue loop unrolling for ks <= 2 (code size vs instruction-level parallelism)
+#endif
 
 // Epilogue of this CTA's reduced slice (rows [rank R, (rank + 1) R) of the tile, R = BM / KS):
 // thread tid owns elements e = rank * PER + tid + NT * i (i < NEL); + Z_p, truncation, store.
-template <int KS>
-__device__ __forceinline__ void slice_store(const SegArgs<uint64_t> &a, int p, int64_t m0, int64_t n0, int rank,
-                                            const uint64_t *red, const uint64_t zpre[ZPF]) {
-    constexpr int PER = BM * BN / KS, NEL = PER / NT;
+template <typename T, int KS>
+__device__ __forceinline__ void slice_store(const SegArgs<T> &a, int p, int64_t m0, int64_t n0, int rank,
+                                            const T *red, const T zpre[ZPF]) {
+    constexpr int PER = BM * BN / KS, NEL = PER / NT, UNR = NEL <= ZPF ? NEL : TCSEG_EPI_UNROLL;
     const int tid = threadIdx.x, party = a.party[p];
-#pragma unroll
+#pragma unroll (UNR)
     for (int i = 0; i < NEL; ++i) {
         const int e = rank * PER + tid + NT * i;
         const int r = e / BN, c = e % BN;
         const int64_t m = m0 + r, n = n0 + c;
         const int64_t off = (m < a.M ? m : a.M - 1) * a.N + (n < a.N ? n : a.N - 1);
-        const uint64_t z = NEL <= ZPF ? zpre[i < ZPF ? i : 0] : ldg(a.Z[p] + off);
-        const uint64_t sum = red[r * RED_PITCH + c];
-        if (m < a.M && n < a.N) a.C[p][off] = trunc_share<uint64_t>(sum + z, party, a.trunc);
+        const T z = !a.Z[p] ? 0 : NEL <= ZPF ? zpre[i < ZPF ? i : 0] : ldg(a.Z[p] + off);
+        const T sum = red[r * RED_PITCH + c];
+        if (m < a.M && n < a.N) a.C[p][off] = trunc_share<T>(sum + z, party, a.trunc);
     }
 }
 
 // The same epilogue, summing the slice's rows straight out of every cluster CTA's partial tile
 // (ld.shared::cluster: distributed shared memory reads, KS loads per element in flight).
-template <int KS>
-__device__ __forceinline__ void slice_sum_store(const SegArgs<uint64_t> &a, int p, int64_t m0, int64_t n0, int rank,
-                                                uint32_t red_u32, const uint64_t zpre[ZPF]) {
-    constexpr int PER = BM * BN / KS, NEL = PER / NT;
+template <typename T, int KS>
+__device__ __forceinline__ void slice_sum_store(const SegArgs<T> &a, int p, int64_t m0, int64_t n0, int rank,
+                                                uint32_t red_u32, const T zpre[ZPF]) {
+    constexpr int PER = BM * BN / KS, NEL = PER / NT, UNR = NEL <= ZPF ? NEL : TCSEG_EPI_UNROLL;
     const int tid = threadIdx.x, party = a.party[p];
     uint32_t peer[KS];
 #pragma unroll
     for (int q = 0; q < KS; ++q) asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(peer[q]) : "r"(red_u32), "r"(q));
-#pragma unroll
+#pragma unroll (UNR)
     for (int i = 0; i < NEL; ++i) {
         const int e = rank * PER + tid + NT * i;
         const int r = e / BN, c = e % BN;
-        const uint32_t off = (uint32_t)(r * RED_PITCH + c) * 8;
-        uint64_t part[KS];
+        const uint32_t off = (uint32_t)(r * RED_PITCH + c) * (uint32_t)sizeof(T);
+        T part[KS];
 #pragma unroll
-        for (int q = 0; q < KS; ++q) asm volatile("ld.shared::cluster.u64 %0, [%1];" : "=l"(part[q]) : "r"(peer[q] + off));
-        uint64_t sum = 0;
+        for (int q = 0; q < KS; ++q) part[q] = ld_dsmem(peer[q] + off, (T *)nullptr);
+        T sum = 0;
 #pragma unroll
         for (int q = 0; q < KS; ++q) sum += part[q];
         const int64_t m = m0 + r, n = n0 + c;
         const int64_t o = (m < a.M ? m : a.M - 1) * a.N + (n < a.N ? n : a.N - 1);
-        const uint64_t z = NEL <= ZPF ? zpre[i < ZPF ? i : 0] : ldg(a.Z[p] + o);
-        if (m < a.M && n < a.N) a.C[p][o] = trunc_share<uint64_t>(sum + z, party, a.trunc);
+        const T z = !a.Z[p] ? 0 : NEL <= ZPF ? zpre[i < ZPF ? i : 0] : ldg(a.Z[p] + o);
+        if (m < a.M && n < a.N) a.C[p][o] = trunc_share<T>(sum + z, party, a.trunc);
     }
 }
 
-#ifndef PSML_TCSEG_RED
-#define PSML_TCSEG_RED 1   // split-K reduction: 0 bulk-copy .add.u64 into the owner CTA, 1 DSMEM reads
-#endif
 
 // grid (total tiles, 1, ks), cluster (1, 1, ks), NTH threads, SMEM_BYTES dynamic shared memory.
-// Warps 0-7 land the raw operand words (cp.async) and split them into limb planes; warp 8 issues
+// Warps 0-7 load the operand words into registers and split them into limb planes; warp 8 issues
 // the MMAs of each limb stage as soon as its `full` barrier completes, so the tensor core works
 // on block i while the producers split block i + 1.
-__global__ void __launch_bounds__(NTH, 1) tc_seg_kernel(const __grid_constant__ Group g) {
+template <typename T>
+__global__ void __launch_bounds__(NTH, 1) tc_seg_kernel(const __grid_constant__ Group<T> g) {
+    constexpr int L = (int)sizeof(T);   // 8-bit limbs per ring element
+#ifndef TCSEG_PD64
+#define TCSEG_PD64 2
+#endif
+#ifndef TCSEG_PD32
+#define TCSEG_PD32 2
+#endif
+    constexpr int PD = L == 8 ? TCSEG_PD64 : TCSEG_PD32;   // K blocks of operand words in flight per producer
     namespace cg = cooperative_groups;
     extern __shared__ __align__(1024) uint8_t smem[];
     uint64_t *empty = (uint64_t *)(smem + PIPE_BYTES);   // limb stage free (MMAs of its block done)
     uint64_t *full = empty + STAGES;                      // limb stage written by all NT producers
     uint64_t *accum = full + STAGES;
-    uint64_t *rbar = accum + 1;   // split-K reduction: peers' partial slices landed
-    uint32_t *tmem_slot = (uint32_t *)(rbar + 1);
+    uint32_t *tmem_slot = (uint32_t *)(accum + 1);
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
 #ifdef TCSEG_TIMING
     uint64_t ts[9];
@@ -219,18 +238,18 @@ __global__ void __launch_bounds__(NTH, 1) tc_seg_kernel(const __grid_constant__ 
 #pragma unroll
     for (int q = 1; q < SEG_MAX_JOBS; ++q)
         if (q < g.njobs && t >= g.tile_begin[q]) jb = q;
-    const SegArgs<uint64_t> &a = g.j[jb];
+    const SegArgs<T> &a = g.j[jb];
     const int64_t tt = t - g.tile_begin[jb];
     const int64_t per_party = (int64_t)g.tiles_m[jb] * g.tiles_n[jb];
     const int p = (int)(tt / per_party);
     const int64_t tp = tt - p * per_party;
     const int64_t m0 = (tp / g.tiles_n[jb]) * BM, n0 = (tp % g.tiles_n[jb]) * BN;
-    const int64_t M = a.M, N = a.N, K = a.K, Kext = 2 * K;
+    const int64_t M = a.M, N = a.N, K = a.K, Kext = g.segs * K;
     const int nkb = (int)((Kext + BK - 1) / BK);
     const int kb0 = (int)blockIdx.z * g.kb_per_split[jb];
     const int kb1 = min(kb0 + g.kb_per_split[jb], nkb);
     const int nblk = kb1 > kb0 ? kb1 - kb0 : 0;
-    const uint64_t *Xp = a.X[p], *Ep = a.E, *Fp = a.F, *Vp = a.V[p];
+    const T *Xp = a.X[p], *Ep = a.E, *Fp = a.F, *Vp = a.V[p];
 
     if (tid == 0) {
         for (int s = 0; s < STAGES; ++s) {
@@ -238,7 +257,6 @@ __global__ void __launch_bounds__(NTH, 1) tc_seg_kernel(const __grid_constant__ 
             mbar_init(smem_u32(&full[s]), NT);
         }
         mbar_init(smem_u32(accum), 1);
-        mbar_init(smem_u32(rbar), 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     if (warp == 1) {
@@ -252,13 +270,13 @@ __global__ void __launch_bounds__(NTH, 1) tc_seg_kernel(const __grid_constant__ 
     TS(1);
     // this CTA's epilogue elements e = rank * per + tid + NT * i (i < 32 / ks): prefetch their
     // Z_p words now (ks >= 4), so the epilogue does not wait on global memory
-    uint64_t zpre[ZPF];
+    T zpre[ZPF];
     {
         const int ks = g.ks, nel = (BM * BN) / ks / NT;
 #pragma unroll
         for (int i = 0; i < ZPF; ++i) {
             zpre[i] = 0;
-            if (nel <= ZPF && i < nel && tid < NT) {
+            if (nel <= ZPF && i < nel && tid < NT && a.Z[p]) {
                 const int e = (int)blockIdx.z * (nel * NT) + tid + NT * i;
                 const int64_t m = m0 + e / BN, n = n0 + e % BN;
                 zpre[i] = ldg(a.Z[p] + (m < M ? m : M - 1) * N + (n < N ? n : N - 1));
@@ -266,86 +284,9 @@ __global__ void __launch_bounds__(NTH, 1) tc_seg_kernel(const __grid_constant__ 
         }
     }
 
-    // stash assignment: A unit = (row ar, 16-k half ac); B unit = (column bn, 8-k quarter bq)
-    const int ar = tid >> 1, ac = tid & 1;
+    // B unit of a producer thread: column bn, 8-k quarter bq of each K block
     const int bn = tid & 63, bq = tid >> 6;
-    // cp.async of one K block's raw words into raw stage rs (zero-filled outside the operands):
-    // 16-byte chunks when the X | E boundary and row starts allow it (K, N even), else 8-byte
-    auto al16 = [](const void *q) { return ((uintptr_t)q & 15) == 0; };
-    const bool a16 = (K % 2) == 0 && al16(Xp) && al16(Ep), b16 = (N % 2) == 0 && al16(Fp) && al16(Vp);
-    auto issue = [&](int kb, int rs) {
-        uint8_t *ra = smem + RAW_OFF + rs * RAW_STAGE_BYTES, *rb = ra + RAW_A_BYTES;
-        const int64_t k0 = (int64_t)kb * BK;
-        if (a16) {
-#pragma unroll
-            for (int u = 0; u < BM * BK / 2 / NT; ++u) {
-                const int c = tid + NT * u, row = c >> 4, kk = (c & 15) * 2;
-                const int64_t m = m0 + row, k = k0 + kk;
-                const bool ok = m < M && k < Kext;
-                const int64_t mc = ok ? m : 0, kc = ok ? k : 0;
-                const uint64_t *src = kc < K ? Xp + mc * K + kc : Ep + mc * K + (kc - K);
-                cp_async16(ra + row * RAW_A_PITCH * 8 + kk * 8, src, ok);
-            }
-        } else {
-#pragma unroll 4
-            for (int u = 0; u < BM * BK / NT; ++u) {
-                const int c = tid + NT * u, row = c >> 5, kk = c & 31;
-                const int64_t m = m0 + row, k = k0 + kk;
-                const bool ok = m < M && k < Kext;
-                const int64_t mc = ok ? m : 0, kc = ok ? k : 0;
-                const uint64_t *src = kc < K ? Xp + mc * K + kc : Ep + mc * K + (kc - K);
-                cp_async8(ra + row * RAW_A_PITCH * 8 + kk * 8, src, ok);
-            }
-        }
-        if (b16) {
-#pragma unroll
-            for (int u = 0; u < BK * BN / 2 / NT; ++u) {
-                const int c = tid + NT * u, kk = c >> 5, nn = (c & 31) * 2;
-                const int64_t k = k0 + kk, n = n0 + nn;
-                const bool ok = k < Kext && n < N;
-                const int64_t kc = ok ? k : 0, ncl = ok ? n : 0;
-                const uint64_t *src = kc < K ? Fp + kc * N + ncl : Vp + (kc - K) * N + ncl;
-                cp_async16(rb + (kk * BN + nn) * 8, src, ok);
-            }
-        } else {
-#pragma unroll 4
-            for (int u = 0; u < BK * BN / NT; ++u) {
-                const int c = tid + NT * u, kk = c >> 6, nn = c & 63;
-                const int64_t k = k0 + kk, n = n0 + nn;
-                const bool ok = k < Kext && n < N;
-                const int64_t kc = ok ? k : 0, ncl = ok ? n : 0;
-                const uint64_t *src = kc < K ? Fp + kc * N + ncl : Vp + (kc - K) * N + ncl;
-                cp_async8(rb + (kk * BN + nn) * 8, src, ok);
-            }
-        }
-    };
-    const int a_off = (((ar >> 3) * 2 + ac) * 128) + (ar & 7) * 16;
     const int b_off = (((bn >> 3) * 2 + (bq >> 1)) * 128) + (bn & 7) * 16 + (bq & 1) * 8;
-    auto stash = [&](int rs, int st) {
-        const uint8_t *ra = smem + RAW_OFF + rs * RAW_STAGE_BYTES, *rb = ra + RAW_A_BYTES;
-        uint8_t *sa = smem + st * STAGE_BYTES, *sb = sa + L * A_TILE;
-        uint64_t va[16], vb[8];
-#pragma unroll
-        for (int j = 0; j < 16; j += 2) {
-            const ulonglong2 v = *(const ulonglong2 *)(ra + ar * RAW_A_PITCH * 8 + (16 * ac + j) * 8);
-            va[j] = v.x;
-            va[j + 1] = v.y;
-        }
-#pragma unroll
-        for (int j = 0; j < 8; ++j) vb[j] = *(const uint64_t *)(rb + ((8 * bq + j) * BN + bn) * 8);
-        uint32_t w[4][8];
-#pragma unroll
-        for (int q = 0; q < 4; ++q) limbs4(va + 4 * q, w[q]);
-#pragma unroll
-        for (int l = 0; l < L; ++l)
-            *(uint4 *)(sa + l * A_TILE + a_off) = make_uint4(w[0][l], w[1][l], w[2][l], w[3][l]);
-        uint32_t u[2][8];
-        limbs4(vb, u[0]);
-        limbs4(vb + 4, u[1]);
-#pragma unroll
-        for (int l = 0; l < L; ++l) *(uint2 *)(sb + l * B_TILE + b_off) = make_uint2(u[0][l], u[1][l]);
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // generic writes -> tensor core
-    };
 
     // Programmatic dependent launch: everything above (barriers, TMEM, Z prefetch -- the dealer's
     // output, complete before the predecessor kernel started) overlapped the predecessor; the
@@ -353,21 +294,101 @@ __global__ void __launch_bounds__(NTH, 1) tc_seg_kernel(const __grid_constant__ 
     pdl_trigger();
     pdl_wait();
     if (warp < NT / 32) {   // producers
-        if (nblk > 0) issue(kb0, 0);
-        cp_async_commit();
-        if (nblk > 1) issue(kb0 + 1, 1);
-        cp_async_commit();
+        // Each thread owns four A units (row u >> 3, 4-k chunk u & 7 of units u = tid + NT i: a warp
+        // reads 4 whole 256-byte rows per instruction, one 32-byte load per unit) and one B unit
+        // (column bn, 8-k quarter bq) of every K block, and loads their words straight into
+        // registers two blocks ahead (double-buffered register sets): a block's words pass through
+        // shared memory once -- as limb planes -- instead of raw words in + out + limb planes.
+        const int64_t bnn = n0 + bn;
+        const bool bcol = bnn < N;
+        auto alv = [](const void *q) { return ((uintptr_t)q & (4 * sizeof(T) - 1)) == 0; };
+        const bool a32 = (K % 4) == 0 && alv(Xp) && alv(Ep);
+        // interior blocks (every row / column inside, the 32 k inside one segment) take a fast path:
+        // precomputed row offsets, no bounds checks, one address add per load
+        const bool rows_full = m0 + BM <= M && a32, cols_full = n0 + BN <= N;
+        int64_t rowoff[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+            const int u = tid + NT * i;
+            rowoff[i] = (m0 + (u >> 3)) * K + 4 * (u & 7);
+        }
+        const int64_t colbase = (int64_t)(8 * bq) * N + bnn;
+        auto load = [&](int kb, T (&va)[16], T (&vb)[8]) {
+            const int64_t k0 = (int64_t)kb * BK;
+            const bool one_seg = k0 + BK <= K || (k0 >= K && k0 + BK <= Kext);
+            if (rows_full && one_seg) {
+                const T *sb = k0 < K ? Xp + k0 : Ep + (k0 - K);
+#pragma unroll
+                for (int i = 0; i < 4; ++i) ld4(sb + rowoff[i], va + 4 * i);
+            } else {
+#pragma unroll
+                for (int i = 0; i < 4; ++i) {
+                    const int u = tid + NT * i, row = u >> 3;
+                    const int64_t m = m0 + row, k = k0 + 4 * (u & 7);
+                    const int64_t mc = m < M ? m : 0;
+                    if (a32) {
+                        if (m < M && k < Kext) {
+                            ld4(k < K ? Xp + mc * K + k : Ep + mc * K + (k - K), va + 4 * i);
+                        } else {
+                            va[4 * i] = va[4 * i + 1] = va[4 * i + 2] = va[4 * i + 3] = 0;
+                        }
+                    } else {
+#pragma unroll
+                        for (int j = 0; j < 4; ++j) {
+                            const int64_t kk = k + j;
+                            va[4 * i + j] = (m < M && kk < Kext) ? ldg(kk < K ? Xp + mc * K + kk : Ep + mc * K + (kk - K)) : 0;
+                        }
+                    }
+                }
+            }
+            if (cols_full && one_seg) {
+                const T *bb = (k0 < K ? Fp + k0 * N : Vp + (k0 - K) * N) + colbase;
+#pragma unroll
+                for (int j = 0; j < 8; ++j) vb[j] = ldg(bb + j * N);
+            } else {
+                const int64_t kbq = k0 + 8 * bq;
+#pragma unroll
+                for (int j = 0; j < 8; ++j) {
+                    const int64_t k = kbq + j;
+                    vb[j] = (bcol && k < Kext) ? ldg(k < K ? Fp + k * N + bnn : Vp + (k - K) * N + bnn) : 0;
+                }
+            }
+        };
+        auto stash_regs = [&](int st, const T (&va)[16], const T (&vb)[8]) {
+            uint8_t *sa = smem + st * STAGE_BYTES, *sb = sa + L * A_TILE;
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+                const int u = tid + NT * i, row = u >> 3, c = u & 7;
+                const int off = (((row >> 3) * 2 + (c >> 2)) * 128) + (row & 7) * 16 + (c & 3) * 4;
+                uint32_t w[L];
+                limbs4(va + 4 * i, w);
+#pragma unroll
+                for (int l = 0; l < L; ++l) *(uint32_t *)(sa + l * A_TILE + off) = w[l];
+            }
+            uint32_t u[2][L];
+            limbs4(vb, u[0]);
+            limbs4(vb + 4, u[1]);
+#pragma unroll
+            for (int l = 0; l < L; ++l) *(uint2 *)(sb + l * B_TILE + b_off) = make_uint2(u[0][l], u[1][l]);
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // generic writes -> tensor core
+        };
+        // PD register sets: block i + PD is loaded as soon as block i is stashed
+        T ra[PD][16], rb[PD][8];
+#pragma unroll
+        for (int d = 0; d < PD; ++d)
+            if (d < nblk) load(kb0 + d, ra[d], rb[d]);
         TS(2);
-        for (int i = 0; i < nblk; ++i) {
-            const int st = i % STAGES, rs = i % RAW_STAGES;
-            cp_async_wait1();                                 // this thread's chunks of block i landed
-            asm volatile("bar.sync 1, %0;" ::"n"(NT) : "memory");   // ... and every producer's
+        auto step = [&](int i, T (&va)[16], T (&vb)[8]) {
+            const int st = i % STAGES;
             if (i >= STAGES) mbar_wait(smem_u32(&empty[st]), (uint32_t)((i / STAGES - 1) & 1));
-            stash(rs, st);                                    // ends with fence.proxy.async
+            stash_regs(st, va, vb);
             asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(&full[st])) : "memory");
-            asm volatile("bar.sync 1, %0;" ::"n"(NT) : "memory");   // raw stage rs read by everyone
-            if (i + 2 < nblk) issue(kb0 + i + 2, rs);
-            cp_async_commit();
+            if (i + PD < nblk) load(kb0 + i + PD, va, vb);
+        };
+        for (int i = 0; i < nblk; i += PD) {
+#pragma unroll
+            for (int d = 0; d < PD; ++d)
+                if (i + d < nblk) step(i + d, ra[d], rb[d]);
         }
     } else if (lane == 0) {   // the MMA warp: 36 limb-pair MMAs per stage into the shift accumulators
         for (int i = 0; i < nblk; ++i) {
@@ -397,8 +418,8 @@ __global__ void __launch_bounds__(NTH, 1) tc_seg_kernel(const __grid_constant__ 
     __syncwarp();
     TS(3);
 
-    // ---- partial tile: sum_s S_s 2^{8s} (u64, exact) -> reduction buffer ----
-    uint64_t *red = (uint64_t *)smem;   // the pipeline region is idle once `accum` completes
+    // ---- partial tile: sum_s S_s 2^{8s} (mod 2^l, exact) -> reduction buffer ----
+    T *red = (T *)smem;   // the pipeline region is idle once `accum` completes
     mbar_wait(smem_u32(accum), 0);
     TS(4);
     fence_after();
@@ -407,7 +428,7 @@ __global__ void __launch_bounds__(NTH, 1) tc_seg_kernel(const __grid_constant__ 
         const uint32_t lane_base = tmem + ((uint32_t)((warp & 3) * 32) << 16);
 #pragma unroll 1
         for (int j0 = (warp >> 2) * (BN / 2); j0 < (warp >> 2) * (BN / 2) + BN / 2; j0 += 16) {
-            uint64_t acc[16];
+            T acc[16];
 #pragma unroll
             for (int j = 0; j < 16; ++j) acc[j] = 0;
             if (nblk > 0) {
@@ -419,68 +440,39 @@ __global__ void __launch_bounds__(NTH, 1) tc_seg_kernel(const __grid_constant__ 
 #pragma unroll
                     for (int u = 0; u < 4; ++u)
 #pragma unroll
-                        for (int j = 0; j < 16; ++j) acc[j] += (uint64_t)r[16 * u + j] << (8 * (s0 + u));
+                        for (int j = 0; j < 16; ++j) acc[j] += (T)r[16 * u + j] << (8 * (s0 + u));
                 }
             }
 #pragma unroll
             for (int j = 0; j < 16; ++j) red[row * RED_PITCH + j0 + j] = acc[j];
         }
     }
-    // ---- split-K reduction by the bulk-copy engine: rows [q R, (q + 1) R) of every CTA's partial
-    // tile (R = BM / ks) are added (cp.reduce.async.bulk .add.u64) into CTA q's copy; CTA q then
-    // runs the epilogue on its fully reduced slice from local shared memory ----
+    // ---- split-K reduction: each CTA sums rows [rank R, (rank + 1) R) (R = BM / ks) of every
+    // cluster CTA's partial tile straight out of their shared memory (DSMEM reads) and runs the
+    // epilogue on that slice ----
     const int ks = g.ks;
     cg::cluster_group cluster = cg::this_cluster();
     const int rank = (int)cluster.block_rank();
-    if (PSML_TCSEG_RED == 1 && ks > 1) {
-        cluster.sync();   // every CTA's partial tile written
-        TS(6);
-        const uint32_t rb = smem_u32(red);
-        if (tid < NT) switch (ks) {
-        case 2: slice_sum_store<2>(a, p, m0, n0, rank, rb, zpre); break;
-        case 4: slice_sum_store<4>(a, p, m0, n0, rank, rb, zpre); break;
-        case 8: slice_sum_store<8>(a, p, m0, n0, rank, rb, zpre); break;
-        default: slice_sum_store<16>(a, p, m0, n0, rank, rb, zpre); break;
-        }
-    } else {
-        const uint32_t slice_bytes = (uint32_t)(BM / ks) * RED_PITCH * 8;
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // red writes -> bulk-copy proxy
-        if (tid == 0 && ks > 1)
-            asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(rbar)),
-                         "r"((uint32_t)(ks - 1) * slice_bytes)
-                         : "memory");
-        fence_before();
-        cluster.sync();   // every partial written, every receiver armed, every pipeline idle
-        TS(6);
-        if (tid == 0 && ks > 1) {
-            const uint32_t base = smem_u32(red), bar = smem_u32(rbar);
-            for (int q = 0; q < ks; ++q) {
-                if (q == rank) continue;
-                const uint32_t src = base + (uint32_t)q * slice_bytes;
-                uint32_t dst, dbar;
-                asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(dst) : "r"(src), "r"(q));
-                asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(dbar) : "r"(bar), "r"(q));
-                asm volatile(
-                    "cp.reduce.async.bulk.shared::cluster.shared::cta.mbarrier::complete_tx::bytes.add.u64 [%0], [%1], "
-                    "%2, [%3];" ::"r"(dst),
-                    "r"(src), "r"(slice_bytes), "r"(dbar)
-                    : "memory");
-            }
-        }
-        if (ks > 1) mbar_wait(smem_u32(rbar), 0);
-        if (tid < NT) switch (ks) {
-        case 1: slice_store<1>(a, p, m0, n0, rank, red, zpre); break;
-        case 2: slice_store<2>(a, p, m0, n0, rank, red, zpre); break;
-        case 4: slice_store<4>(a, p, m0, n0, rank, red, zpre); break;
-        case 8: slice_store<8>(a, p, m0, n0, rank, red, zpre); break;
-        default: slice_store<16>(a, p, m0, n0, rank, red, zpre); break;
-        }
+    cluster.sync();   // every CTA's partial tile written
+    TS(6);
+    if (tid < NT) switch (ks) {
+    case 1: slice_store<T, 1>(a, p, m0, n0, rank, red, zpre); break;
+    case 2: slice_sum_store<T, 2>(a, p, m0, n0, rank, smem_u32(red), zpre); break;
+    case 4: slice_sum_store<T, 4>(a, p, m0, n0, rank, smem_u32(red), zpre); break;
+    case 8: slice_sum_store<T, 8>(a, p, m0, n0, rank, smem_u32(red), zpre); break;
+    default: slice_sum_store<T, 16>(a, p, m0, n0, rank, smem_u32(red), zpre); break;
     }
     cluster.sync();   // peers' shared memory stays alive until every CTA has read it
     TS(7);
     if (warp == 1) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tmem));
     TS(8);
-#ifdef TCSEG_TIMING
+#ifdef TCSEG_TIMING_ALL
+    if (tid == 0) {
+        uint32_t smid;
+        asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+        printf("tcsegall %d %d %u %llu %llu\n", (int)blockIdx.x, (int)blockIdx.z, smid, ts[0], ts[8]);
+    }
+#elif defined(TCSEG_TIMING)
     if (tid == 0 && (blockIdx.x == 0 || blockIdx.x == gridDim.x - 1) && blockIdx.z < 2)
         printf("tcseg grid %d blk %d z %d nblk %d: prologue %llu load0 %llu mma %llu accum %llu red %llu reduce %llu end %llu total %llu ns\n",
                (int)gridDim.x, (int)blockIdx.x, (int)blockIdx.z, nblk, ts[1] - ts[0], ts[2] - ts[1], ts[3] - ts[2],
@@ -508,14 +500,19 @@ bool tc_seg_enabled() {
 // psml_options.pdl = 0 disables programmatic dependent launch of the GEMMs after their producers.
 bool pdl_enabled() { return cur_opts().pdl != 0; }
 
-psml_status tc_seg_group(const SegArgs<uint64_t> *jobs, int njobs, cudaStream_t stream, int sm_count) {
+template <typename T>
+static psml_status tc_seg_group_t(const SegArgs<T> *jobs, int njobs, cudaStream_t stream, int sm_count, int segs,
+                                  int fill) {
     using namespace tcseg;
     if (njobs < 1 || njobs > SEG_MAX_JOBS) return fail(PSML_ERR_INVALID, "tc seg group: 1..4 jobs");
     static int attr_done = 0;
     static int max_ks = 8;
     if (!attr_done) {
-        PSML_CUDA_TRY(cudaFuncSetAttribute(tc_seg_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM_BYTES));
-        if (cudaFuncSetAttribute(tc_seg_kernel, cudaFuncAttributeNonPortableClusterSizeAllowed, 1) == cudaSuccess) {
+        PSML_CUDA_TRY(cudaFuncSetAttribute(tcseg::tc_seg_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM_BYTES));
+#ifdef TCSEG_CARVEOUT
+        PSML_CUDA_TRY(cudaFuncSetAttribute(tcseg::tc_seg_kernel<T>, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
+#endif
+        if (cudaFuncSetAttribute(tcseg::tc_seg_kernel<T>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1) == cudaSuccess) {
             cudaLaunchConfig_t q = {};
             q.gridDim = dim3(MAX_KS, 1, MAX_KS);
             q.blockDim = dim3(NTH);
@@ -526,36 +523,41 @@ psml_status tc_seg_group(const SegArgs<uint64_t> *jobs, int njobs, cudaStream_t 
             q.attrs = at;
             q.numAttrs = 1;
             int n = 0;
-            if (cudaOccupancyMaxActiveClusters(&n, tc_seg_kernel, &q) == cudaSuccess && n >= 4) max_ks = MAX_KS;
+            if (cudaOccupancyMaxActiveClusters(&n, tcseg::tc_seg_kernel<T>, &q) == cudaSuccess && n >= 4) max_ks = MAX_KS;
         }
         cudaGetLastError();
         attr_done = 1;
     }
-    Group g{};
+    Group<T> g{};
     int64_t tiles = 0;
     int nkb_max = 1;
     double work = 0;
     for (int q = 0; q < njobs; ++q) {
-        const SegArgs<uint64_t> &j = jobs[q];
-        if (2 * j.K > 16384) return fail(PSML_ERR_UNSUPPORTED, "tc seg: K' > 16384 per product");
+        const SegArgs<T> &j = jobs[q];
+        // l = 64: K' <= 2^14 per CTA keeps S_0..S_3 exact in s32 (every shift wraps harmlessly mod 2^32 at l = 32)
+        if (sizeof(T) == 8 && segs * j.K > 16384) return fail(PSML_ERR_UNSUPPORTED, "tc seg: K' > 16384 per product");
         g.j[q] = j;
         g.tiles_m[q] = (int)((j.M + BM - 1) / BM);
         g.tiles_n[q] = (int)((j.N + BN - 1) / BN);
         g.tile_begin[q] = tiles;
         tiles += (int64_t)g.tiles_m[q] * g.tiles_n[q] * j.nparty;
-        nkb_max = std::max(nkb_max, (int)((2 * j.K + BK - 1) / BK));
-        work += (double)j.M * j.N * 2 * j.K * j.nparty;
+        nkb_max = std::max(nkb_max, (int)((segs * j.K + BK - 1) / BK));
+        work += (double)j.M * j.N * segs * j.K * j.nparty;
     }
     g.tile_begin[njobs] = tiles;
     g.njobs = njobs;
-    // K split: double ks while the grid stays within 1/PSML_TCSEG_FILL of the SMs (default 2: the
-    // rest stays with the dealer branch) and each split keeps >= 2 K blocks
-    const int fill = PSML_TCSEG_FILL;
+    g.segs = segs;
+    // K split: double ks while the grid stays within 1/fill of the SMs (training step: 2, the rest
+    // stays with the dealer branch; stand-alone products: 1) and each split keeps >= 2 K blocks
     int ks = 1;
-    while (ks < max_ks && tiles * ks * 2 * fill <= 2 * sm_count && nkb_max >= ks * 2) ks *= 2;
+    if (fill > 1) {   // training step (measured: up to 2 sm_count / fill CTAs)
+        while (ks < max_ks && tiles * ks * 2 * fill <= 2 * sm_count && nkb_max >= ks * 2) ks *= 2;
+    } else {          // stand-alone: the whole grid in one wave of one-CTA-per-SM clusters
+        while (ks < max_ks && tiles * ks * 2 <= sm_count && nkb_max >= ks * 2) ks *= 2;
+    }
     g.ks = ks;
     for (int q = 0; q < njobs; ++q) {
-        const int nkb = (int)((2 * jobs[q].K + BK - 1) / BK);
+        const int nkb = (int)((segs * jobs[q].K + BK - 1) / BK);
         g.kb_per_split[q] = (nkb + ks - 1) / ks;
     }
     cudaLaunchConfig_t cfg = {};
@@ -577,9 +579,80 @@ psml_status tc_seg_group(const SegArgs<uint64_t> *jobs, int njobs, cudaStream_t 
         cfg.numAttrs = 3;
     }
     ProfScope prof(PROF_TC, stream, work);
-    PSML_CUDA_TRY(cudaLaunchKernelEx(&cfg, tcseg::tc_seg_kernel, g));
+    PSML_CUDA_TRY(cudaLaunchKernelEx(&cfg, tcseg::tc_seg_kernel<T>, g));
     g_launches.fetch_add(1, std::memory_order_relaxed);
     return PSML_OK;
 }
+
+psml_status tc_seg_group(const SegArgs<uint64_t> *jobs, int njobs, cudaStream_t stream, int sm_count, int segs,
+                         int fill) {
+    return tc_seg_group_t<uint64_t>(jobs, njobs, stream, sm_count, segs, fill);
+}
+
+// ------------------------------------------------------------------------------------------------
+// Stand-alone products on the same kernel (BASELINE config 5 at n <= 2048, psml_ring_gemm and the
+// co-resident psml_secure_matmul): the limb-plane kernels of gemm_tc.cu need a split pass, a
+// split-K memset and a finalize launch around a grid of few 128 x 128 tiles at these sizes; here
+// one launch (plain) or two (Beaver: one mask + open pass, then the Eq. 8 product) cover them,
+// with the K split over a cluster filling the whole GPU.
+// ------------------------------------------------------------------------------------------------
+bool tc_seg_small(int l, int64_t M, int64_t Kext, int64_t N, int nparty, int sm_count) {
+    const int mode = cur_opts().tc_small;   // psml_options.tc_small
+    if (mode == 0 || !tc_seg_enabled() || (l == 64 && Kext > 16384) || M <= 0 || N <= 0) return false;
+    if (mode == 2) return true;
+    // auto: the output tiles fit one wave (measured, tools/tc_small_ab.py: 512^3 plain 44 -> 20 us,
+    // 1024^3 plain 93 -> 64 us; Beaver 1024^3 (256 tiles, two waves) is faster on the limb planes)
+    using namespace tcseg;
+    return ((M + BM - 1) / BM) * ((N + BN - 1) / BN) * nparty <= sm_count;
+}
+
+template <typename T>
+psml_status tc_seg_plain(const T *A, const T *B, int64_t M, int64_t K, int64_t N, T *C, cudaStream_t s, int sm_count) {
+    SegArgs<T> a{};
+    a.X[0] = A; a.F = B; a.C[0] = C;
+    a.M = M; a.N = N; a.K = K; a.trunc = 0; a.nparty = 1;
+    return tc_seg_group_t<T>(&a, 1, s, sm_count, 1, 1);
+}
+
+template <typename T>
+size_t tc_seg_beaver_ws_bytes(int64_t M, int64_t K, int64_t N) { return sizeof(T) * (size_t)(2 * M * K + K * N) + 512; }
+
+template <typename T>
+psml_status tc_seg_beaver(const T *const A[2], const T *const B[2], const T *const U[2], const T *const V[2],
+                          const T *const Z[2], int64_t M, int64_t K, int64_t N, int flags, int trunc, T *const C[2],
+                          void *ws, size_t ws_bytes, cudaStream_t s, int sm_count) {
+    if (ws_bytes < tc_seg_beaver_ws_bytes<T>(M, K, N)) return fail(PSML_ERR_NOMEM, "tc seg Beaver workspace too small");
+    T *E = (T *)(((uintptr_t)ws + 255) & ~(uintptr_t)255), *X1 = E + M * K, *F = X1 + M * K;
+    // Eqs. 4-5 for both parties in one pass: E = (A_0 - U_0) + (A_1 - U_1), X_1 = E + U_1,
+    // F = (B_0 - V_0) + (B_1 - V_1) (op layouts; transposed sources through shared memory)
+    OpenList<T> L{};
+    const int tA = (flags & PSML_TRANS_A) ? 1 : 0, tB = (flags & PSML_TRANS_B) ? 1 : 0;
+    L.j[0] = {{A[0], A[1]}, {U[0], U[1]}, E, X1, U[1], (T)1, M, K, tA};
+    L.j[1] = {{B[0], B[1]}, {V[0], V[1]}, F, nullptr, nullptr, (T)1, K, N, tB};
+    L.n = 2;
+    L.tile_begin[0] = 0;
+    L.tile_begin[1] = ((M + 31) / 32) * ((K + 31) / 32);
+    L.tile_begin[2] = L.tile_begin[1] + ((K + 31) / 32) * ((N + 31) / 32);
+    {
+        ProfScope prof(PROF_MASK, s, 3.0 * 8 * 2 * (M * K + K * N));
+        PSML_CUDA_TRY(launch_pdl(open_list_kernel<T>, dim3((unsigned)L.tile_begin[2]), dim3(32, 8), s, L));
+        PSML_LAUNCH_CHECK();
+    }
+    // Eq. 8 (BJ form): C_p = [X_p | E] . [F ; V_p] + Z_p, X_0 = U_0, then truncation
+    SegArgs<T> a{};
+    a.X[0] = U[0]; a.X[1] = X1; a.E = E; a.F = F;
+    for (int p = 0; p < 2; ++p) { a.V[p] = V[p]; a.Z[p] = Z[p]; a.C[p] = C[p]; a.party[p] = p; }
+    a.M = M; a.N = N; a.K = K; a.trunc = trunc; a.nparty = 2;
+    return tc_seg_group_t<T>(&a, 1, s, sm_count, 2, 1);
+}
+
+#define PSML_TCSEG_INST(T)                                                                                        \
+    template psml_status tc_seg_plain<T>(const T *, const T *, int64_t, int64_t, int64_t, T *, cudaStream_t, int); \
+    template size_t tc_seg_beaver_ws_bytes<T>(int64_t, int64_t, int64_t);                                        \
+    template psml_status tc_seg_beaver<T>(const T *const[2], const T *const[2], const T *const[2], const T *const[2], \
+                                          const T *const[2], int64_t, int64_t, int64_t, int, int, T *const[2], void *, \
+                                          size_t, cudaStream_t, int);
+PSML_TCSEG_INST(uint64_t)
+PSML_TCSEG_INST(uint32_t)
 
 }  // namespace psml

@@ -39,7 +39,8 @@ class Options(ctypes.Structure):
     """psml_options (include/psml.h): explicit per-context execution options."""
     _fields_ = [(n, i32) for n in ("seg_backend", "pdl", "fused_open", "fused_step", "fused_dealer",
                                     "deal_split", "deal_after", "gradw_branch", "simt_cluster",
-                                    "rows_kernel", "msb_chain", "conv_gw", "split_fused", "deal_on_launch")]
+                                    "rows_kernel", "msb_chain", "conv_gw", "split_fused", "deal_on_launch",
+                                    "tc_small")]
 
 
 # Test-harness convenience of the BINDING (the library reads no environment): PSML_* variables
@@ -60,6 +61,7 @@ _ENV_OPTIONS = {
     "PSML_CONV_GW": ("conv_gw", {"generic": 0, "image": 1}),
     "PSML_SPLIT_FUSED": ("split_fused", {"0": 0, "1": 1}),
     "PSML_DEAL_ON_LAUNCH": ("deal_on_launch", {"0": 0, "1": 1}),
+    "PSML_TC_SMALL": ("tc_small", {"0": 0, "1": 1, "2": 2}),
 }
 
 

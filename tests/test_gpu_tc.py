@@ -3,7 +3,9 @@
 Covers single and multiple tiles, ragged M/N/K tails (zero-padded limb planes), split-K with
 atomic partials, the l = 64 exactness limit (K' > 16512 forces exact chunks; all-ones operands
 are the worst case for the int32 shift accumulators), the dealer's Z = U.V and the Beaver
-product with its fused open + Z_i + truncation epilogue.
+product with its fused open + Z_i + truncation epilogue.  Each ring runs twice: on the limb-plane
+kernels (psml_options.tc_small = 0) and on the in-kernel limb-split kernel (tc_small = 2; l = 64
+wherever K' <= 16384, l = 32 always; one-segment plain products, cluster split-K over the GPU).
 """
 import numpy as np
 import pytest
@@ -21,9 +23,11 @@ def P():
     return psml
 
 
-@pytest.fixture(scope="module", params=[64, 32])
+@pytest.fixture(scope="module", params=[(64, 0), (64, 2), (32, 0), (32, 2)],
+                ids=["l64-planes", "l64-split", "l32-planes", "l32-split"])
 def tctx(P, request):
-    c = P.Ctx(l=request.param, frac_bits=13, backend=2)
+    l, small = request.param
+    c = P.Ctx(l=l, frac_bits=13, backend=2, options={"tc_small": small})
     yield c
     c.close()
 
@@ -34,7 +38,7 @@ def _rand(orc, l, n, salt):
 
 @pytest.mark.parametrize("shape", [(128, 32, 64), (128, 64, 128), (1, 1, 1), (130, 33, 65),
                                    (256, 100, 130), (300, 777, 200), (512, 512, 512),
-                                   (128, 4000, 64), (1000, 96, 1000)])
+                                   (128, 4000, 64), (1000, 96, 1000), (640, 2048, 384), (2048, 1024, 2048)])
 def test_tc_ring_gemm_bitexact(P, orc, tctx, shape):
     l = tctx.l
     M, K, N = shape
@@ -69,7 +73,7 @@ def test_tc_triplet_gen(P, orc, tctx, shape):
 
 
 @pytest.mark.parametrize("shape,flags", [((128, 64, 128), 0), ((256, 200, 192), 0), ((300, 130, 260), 3),
-                                         ((512, 784, 128), 1), ((128, 9000, 64), 0)])
+                                         ((512, 784, 128), 1), ((128, 9000, 64), 0), ((1024, 1000, 1100), 2)])
 def test_tc_beaver_matmul_bitexact(P, orc, tctx, shape, flags):
     l = tctx.l
     M, K, N = shape
