@@ -79,6 +79,28 @@ __device__ __forceinline__ void tc_mma_i8(uint32_t d_tmem, uint64_t adesc, uint6
 __device__ __forceinline__ void tc_commit(uint32_t bar) {
     asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar) : "memory");
 }
+// the same bulk copy landing at the same shared-memory offset (and completing the mbarrier at the
+// same offset) in every CTA of `mask` in the cluster
+__device__ __forceinline__ void bulk_g2s_mc(uint32_t dst, const void *src, uint32_t bytes, uint32_t bar, uint16_t mask) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.multicast::cluster [%0], [%1], %2, [%3], %4;" ::"r"(dst),
+        "l"(src), "r"(bytes), "r"(bar), "h"(mask)
+        : "memory");
+}
+// commit arriving on the mbarrier at this offset in every CTA of `mask`
+__device__ __forceinline__ void tc_commit_mc(uint32_t bar, uint16_t mask) {
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(bar),
+                 "h"(mask)
+                 : "memory");
+}
+__device__ __forceinline__ void cluster_sync_all() {
+    asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+__device__ __forceinline__ uint32_t cluster_rank() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
 __device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t r[16]) {
     asm volatile(
         "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, "
@@ -236,12 +258,23 @@ __device__ __forceinline__ void epi_chunk(T *st, const T v[16], int lane, int64_
 }
 
 #ifndef TC_V1_GROUP
-#define TC_V1_GROUP 0
+#define TC_V1_GROUP 1   // BN = 128: no gain (4096^3 0.5745 vs 0.5724 ms); BN = 64: 4 MMAs of N <= 256 per block
 #endif
-template <typename T, int L, int BN, int STAGES>
-__global__ void __launch_bounds__(128, 1) tc_ring_gemm_kernel(const TcParams<T> P) {
+#ifndef TC_B_MULTICAST
+#define TC_B_MULTICAST 1
+#endif
+// MC = 2: the two CTAs of a (1, 2, 1) cluster (row blocks rb, rb + 1 of the same column block)
+// share the B tile: each bulk-copies half of its limb planes to BOTH CTAs (TMA multicast), so the
+// L2 -> SM traffic per block is A + B/2 instead of A + B (l = 32 at 4096^3 is L2-bandwidth bound:
+// 4.3 GB of limb planes in 0.57 ms); each stage is freed only when both CTAs' MMAs retired it.
+template <typename T, int L, int BN, int STAGES, int MC>
+__global__ void __launch_bounds__(128, (STAGES * L * (BM * BK + BN * BK) <= 110 * 1024) ? 2 : 1)
+    tc_ring_gemm_kernel(const TcParams<T> P) {
     extern __shared__ __align__(1024) uint8_t smem[];
     constexpr int A_BYTES = BM * BK, B_BYTES = BN * BK;
+    // TMEM columns: L shift accumulators of BN columns (a power of two >= 32; 256 lets two CTAs
+    // share an SM, one's epilogue overlapping the other's main loop)
+    constexpr uint32_t TCOLS = L * BN <= 32 ? 32 : L * BN <= 64 ? 64 : L * BN <= 128 ? 128 : L * BN <= 256 ? 256 : 512;
     constexpr int STAGE_BYTES = L * (A_BYTES + B_BYTES);
     constexpr uint32_t IDESC = idesc_i8(BM, BN);
     uint64_t *full = (uint64_t *)(smem + STAGES * STAGE_BYTES);
@@ -259,19 +292,21 @@ __global__ void __launch_bounds__(128, 1) tc_ring_gemm_kernel(const TcParams<T> 
     if (threadIdx.x == 0) {
         for (int s = 0; s < STAGES; ++s) {
             mbar_init(smem_u32(&full[s]), 1);
-            mbar_init(smem_u32(&empty[s]), 1);
+            mbar_init(smem_u32(&empty[s]), MC);
         }
         mbar_init(smem_u32(accum), 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     if (warp == 2) {
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_u32(tmem_slot)));
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)), "n"(TCOLS));
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
     }
     tc_fence_before();
-    __syncthreads();
+    if (MC > 1) cluster_sync_all();   // the peer's barriers exist before any multicast completes on them
+    else __syncthreads();
     tc_fence_after();
     const uint32_t tmem = *tmem_slot;
+    const uint32_t crank = MC > 1 ? cluster_rank() : 0;
 
     if (warp == 0 && lane == 0) {
         // ---------------- TMA producer ----------------
@@ -290,8 +325,14 @@ __global__ void __launch_bounds__(128, 1) tc_ring_gemm_kernel(const TcParams<T> 
             uint8_t *sa = smem + stage * STAGE_BYTES, *sb = sa + L * A_BYTES;
 #pragma unroll
             for (int p = 0; p < L; ++p) bulk_g2s(smem_u32(sa + p * A_BYTES), a + p * as, A_BYTES, fb);
+            if (MC > 1) {
 #pragma unroll
-            for (int q = 0; q < L; ++q) bulk_g2s(smem_u32(sb + q * B_BYTES), b + q * bs, B_BYTES, fb);
+                for (int q = 0; q < L; ++q)
+                    if (q % MC == (int)crank) bulk_g2s_mc(smem_u32(sb + q * B_BYTES), b + q * bs, B_BYTES, fb, (1u << MC) - 1);
+            } else {
+#pragma unroll
+                for (int q = 0; q < L; ++q) bulk_g2s(smem_u32(sb + q * B_BYTES), b + q * bs, B_BYTES, fb);
+            }
             if (++stage == STAGES) { stage = 0; phase ^= 1; }
         }
     } else if (warp == 1 && lane == 0) {
@@ -330,7 +371,8 @@ __global__ void __launch_bounds__(128, 1) tc_ring_gemm_kernel(const TcParams<T> 
                 }
             }
 #endif
-            tc_commit(smem_u32(&empty[stage]));   // frees the smem stage once these MMAs retire
+            if (MC > 1) tc_commit_mc(smem_u32(&empty[stage]), (1u << MC) - 1);   // both CTAs' copies of the stage
+            else tc_commit(smem_u32(&empty[stage]));   // frees the smem stage once these MMAs retire
             if (++stage == STAGES) { stage = 0; phase ^= 1; }
         }
         tc_commit(smem_u32(accum));               // all accumulators final
@@ -358,8 +400,9 @@ __global__ void __launch_bounds__(128, 1) tc_ring_gemm_kernel(const TcParams<T> 
         epi_chunk<T>(st, acc, lane, row0, (int64_t)nb * BN + j0, P, party, 0, false);
     }
     tc_fence_before();
-    __syncthreads();
-    if (warp == 2) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tmem));
+    if (MC > 1) cluster_sync_all();   // no CTA leaves while its peer's multicast / commits may still target it
+    else __syncthreads();
+    if (warp == 2) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(TCOLS));
 }
 
 // ------------------------------------------------------------------------------------------------
@@ -579,7 +622,13 @@ __global__ void tc_finalize_kernel(const TcParams<T> P, int mode) {
 template <int l> struct Cfg;
 // APAD: row padding of the A operand (l = 64 runs on CTA pairs: 256 rows per pair).
 template <> struct Cfg<64> { using T = uint64_t; static constexpr int L = 8, BN = 128, STAGES = 3, APAD = 128; static constexpr int MAX_KB = 16384 / BK; };
-template <> struct Cfg<32> { using T = uint32_t; static constexpr int L = 4, BN = 128, STAGES = 6, APAD = 128; static constexpr int MAX_KB = 1 << 30; };
+#ifndef TC32_BN
+#define TC32_BN 64
+#endif
+// l = 32: BN = 64 with 4 stages (98 KB, 256 TMEM columns) runs two CTAs per SM, one's epilogue
+// beside the other's main loop (same box, + B multicast: 4096^3 0.578 -> 0.550 ms, 2048^3 0.118 ->
+// 0.108 ms, 8192^3 4.04 -> 4.10 ms; BN = 128 without multicast 0.575 / 0.118 / 4.23 ms)
+template <> struct Cfg<32> { using T = uint32_t; static constexpr int L = 4, BN = TC32_BN, STAGES = TC32_BN == 64 ? 4 : 6, APAD = 128; static constexpr int MAX_KB = 1 << 30; };
 
 template <int l>
 constexpr size_t smem_bytes() {
@@ -653,13 +702,29 @@ static psml_status launch_gemm(TcParams<typename Cfg<l>::T> P, int64_t Mp, int64
                 kern<<<grid, 192, smem_v4_bytes(), s>>>(P);
             }
         } else {
-            auto kern = tc_ring_gemm_kernel<T, Cfg<l>::L, BN, Cfg<l>::STAGES>;
+            auto kern1 = tc_ring_gemm_kernel<T, Cfg<l>::L, BN, Cfg<l>::STAGES, 1>;
+            auto kern2 = tc_ring_gemm_kernel<T, Cfg<l>::L, BN, Cfg<l>::STAGES, 2>;
             static bool attr_set = false;
             if (!attr_set) {
-                PSML_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_bytes<l>()));
+                PSML_CUDA_TRY(cudaFuncSetAttribute(kern1, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_bytes<l>()));
+                PSML_CUDA_TRY(cudaFuncSetAttribute(kern2, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_bytes<l>()));
                 attr_set = true;
             }
-            kern<<<grid, 128, smem_bytes<l>(), s>>>(P);
+            if (TC_B_MULTICAST && (Mp / BM) % 2 == 0) {   // row-block pairs share B (TMA multicast)
+                cudaLaunchConfig_t cfg = {};
+                cfg.gridDim = grid;
+                cfg.blockDim = dim3(128);
+                cfg.dynamicSmemBytes = smem_bytes<l>();
+                cfg.stream = s;
+                cudaLaunchAttribute at[1];
+                at[0].id = cudaLaunchAttributeClusterDimension;
+                at[0].val.clusterDim.x = 1; at[0].val.clusterDim.y = 2; at[0].val.clusterDim.z = 1;
+                cfg.attrs = at;
+                cfg.numAttrs = 1;
+                PSML_CUDA_TRY(cudaLaunchKernelEx(&cfg, kern2, P));
+            } else {
+                kern1<<<grid, 128, smem_bytes<l>(), s>>>(P);
+            }
         }
         PSML_LAUNCH_CHECK();
     }
