@@ -120,6 +120,10 @@ struct psml_model_s {
     int64_t word_next = -1;            // value *step_dev holds once the last enqueued pipelined
                                        // replay completes (it advances the word itself); -1 unknown
     cudaGraphExec_t graph[2] = {nullptr, nullptr};  // captured step(s) (psml_model_capture_step)
+    cudaGraph_t graph_tmpl[2] = {nullptr, nullptr};  // their templates (the share node's handle lives there)
+    cudaGraphNode_t share_node[2] = {nullptr, nullptr};   // the client's encode + share, first online node
+    bool share_live[2] = {false, false};              // the node holds a real batch's job (else a no-op)
+    unsigned share_grid = 0;
     int graph_flags = 0;
     int64_t graph_kernels = 0;
     cudaStream_t side = nullptr;       // dealer branch inside the pipelined graph
@@ -1730,8 +1734,10 @@ psml_status psml_model_destroy(psml_model model) {
     PSML_CTX_OPTS(model ? model->ctx : nullptr);
     if (!model) return PSML_OK;
     cudaDeviceSynchronize();
-    for (int g = 0; g < 2; ++g)
+    for (int g = 0; g < 2; ++g) {
         if (model->graph[g]) cudaGraphExecDestroy(model->graph[g]);
+        if (model->graph_tmpl[g]) cudaGraphDestroy(model->graph_tmpl[g]);
+    }
     if (model->side) cudaStreamDestroy(model->side);
     if (model->ev_fork) cudaEventDestroy(model->ev_fork);
     if (model->hi) cudaStreamDestroy(model->hi);
@@ -1982,140 +1988,6 @@ static psml_status party_reduce_update(psml_model_s *m, int party, psml_dp dp, c
 // side stream (fork/join inside the capture), reading the step word = step + 1.
 static bool use_prio() { return true; }   // stream priorities in the pipelined graph (865K -> 914K)
 
-static psml_status capture_one(psml_model_s *m, int pool, const T *const X[2], const T *const Y[2], int flags,
-                               cudaStream_t s, cudaGraphExec_t *out, int64_t *kernels) {
-    const bool pipelined = (flags & 4) != 0;
-    const bool prio = pipelined && use_prio();
-    PSML_CUDA_TRY(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
-    psml_status st = PSML_OK;
-    cudaStream_t on = s;   // stream of the online phase
-    if (pipelined) {
-        if (cudaEventRecord(m->ev_fork, s) != cudaSuccess || cudaStreamWaitEvent(m->side, m->ev_fork, 0) != cudaSuccess)
-            st = fail(PSML_ERR_CUDA, "graph fork failed");
-        if (st == PSML_OK && prio) {
-            if (cudaStreamWaitEvent(m->hi, m->ev_fork, 0) != cudaSuccess) st = fail(PSML_ERR_CUDA, "graph fork failed");
-            on = m->hi;
-        }
-        const int after = cur_opts().deal_after;   // default 1: after the step-start open
-        // models without the fused step (the CNN) run large kernels that fill the GPU: their
-        // dealer forks at the start of the step (measured: 51.6K vs 49.4K samples/s forked after)
-        m->deal_after = (fused_eligible(m) && m->cap_party < 0) ? after : 0;
-        m->deal_stage = 0;
-        m->deal_on_launch = m->deal_after > 0 && cur_opts().deal_on_launch != 0;
-        if (m->deal_on_launch) m->deal_after = 2;   // the fork point right after the first product
-        m->fork_event_armed = false;
-        if (st == PSML_OK && m->deal_after == 0) {
-            st = deal_pool(m, 1 - pool, 0, false, m->side, deal_s2(m));
-            if (st == PSML_OK) advance_word_kernel<<<1, 1, 0, m->side>>>(m->step_dev);
-            if (st == PSML_OK && cudaEventRecord(m->ev_join, m->side) != cudaSuccess)
-                st = fail(PSML_ERR_CUDA, "graph join record failed");
-        } else {
-            m->deal_pending_pool = 1 - pool;   // forked from the online chain (deal_fork_point)
-        }
-    } else if (flags & 1) {
-        st = deal_pool(m, pool, 0, false, s);
-    }
-    m->pool = pool;
-    const int pp = m->cap_party;
-    if (st == PSML_OK) {
-        if (pp >= 0) {
-            PartyRun r{m, pp, m->cap_xport, on};
-            st = party_forward_backward(r, X[pp], Y[pp]);
-        } else {
-            st = forward_backward(m, X, Y, on);
-        }
-    }
-    if (st == PSML_OK) st = deal_fork_point(m, on, true);   // not forked yet: fork here
-    m->deal_pending_pool = -1;
-    if (st == PSML_OK && (flags & 2)) {
-        m->grads_ready = true;
-        st = pp >= 0 ? party_reduce_update(m, pp, m->cap_dp, on) : psml_train_apply_update(m, 0, (psml_stream)on);
-    }
-    if (prio && st == PSML_OK &&
-        (cudaEventRecord(m->ev_hi, m->hi) != cudaSuccess || cudaStreamWaitEvent(s, m->ev_hi, 0) != cudaSuccess))
-        st = fail(PSML_ERR_CUDA, "graph join failed");
-    if (pipelined && st == PSML_OK && cudaStreamWaitEvent(s, m->ev_join, 0) != cudaSuccess)
-        st = fail(PSML_ERR_CUDA, "graph join failed");
-    cudaGraph_t g = nullptr;
-    cudaError_t e = cudaStreamEndCapture(s, &g);
-    if (st != PSML_OK) {
-        if (g) cudaGraphDestroy(g);
-        return st;
-    }
-    if (e != cudaSuccess) return fail(PSML_ERR_CUDA, std::string("graph capture: ") + cudaGetErrorString(e));
-    size_t nn = 0;
-    cudaGraphGetNodes(g, nullptr, &nn);
-    std::vector<cudaGraphNode_t> nodes(nn);
-    if (nn) cudaGraphGetNodes(g, nodes.data(), &nn);
-    *kernels = 0;
-    for (auto nd : nodes) {
-        cudaGraphNodeType t;
-        if (cudaGraphNodeGetType(nd, &t) == cudaSuccess && t == cudaGraphNodeTypeKernel) ++*kernels;
-    }
-    // kernel nodes keep the priority of the stream they were captured on
-    e = cudaGraphInstantiateWithFlags(out, g, cudaGraphInstantiateFlagUseNodePriority);
-    cudaGraphDestroy(g);
-    if (e != cudaSuccess) return fail(PSML_ERR_CUDA, std::string("graph instantiate: ") + cudaGetErrorString(e));
-    return PSML_OK;
-}
-
-static psml_status capture_common(psml_model m, const void *const X[2], const void *const Y[2], int32_t flags,
-                                  psml_stream stream) {
-    if (flags & ~15) return fail(PSML_ERR_INVALID, "flags: bit 0 dealer, bit 1 update, bit 2 pipelined dealer, bit 3 reuse");
-    if ((flags & 8) && (flags & 5)) return fail(PSML_ERR_INVALID, "flag bit 3 (material reuse) only applies without a dealer");
-    cudaStream_t s = (cudaStream_t)stream;
-    if (s == nullptr) return fail(PSML_ERR_INVALID, "capture needs a non-default stream");
-    for (int g = 0; g < 2; ++g)
-        if (m->graph[g]) {
-            cudaGraphExecDestroy(m->graph[g]);
-            m->graph[g] = nullptr;
-        }
-    const int prof = g_prof_cls.exchange(-1);   // no profiling events inside the graphs
-    m->word_next = -1;
-    psml_status st = PSML_OK;
-    // one graph per dealer pool, except when the graph deals its own pool 0 (flags bit 0 only)
-    // or replays one pool on purpose (bit 3, benchmark-only material reuse)
-    const bool per_pool = (flags & 4) || !(flags & 9);
-    const int ngraphs = per_pool ? 2 : 1;
-    for (int g = 0; g < ngraphs && st == PSML_OK; ++g)
-        st = capture_one(m, per_pool ? g : 0, (const T *const *)X, (const T *const *)Y, flags, s, &m->graph[g],
-                         &m->graph_kernels);
-    g_prof_cls.store(prof);
-    if (st != PSML_OK) return st;
-    m->graph_flags = flags;
-    for (int i = 0; i < 2; ++i) { m->cap_X[i] = X[i]; m->cap_Y[i] = Y[i]; }
-    return PSML_OK;
-}
-
-psml_status psml_model_capture_step(psml_model m, const void *const X[2], const void *const Y[2], int32_t flags,
-                                   psml_stream stream) {
-    PSML_CTX_OPTS(m ? m->ctx : nullptr);
-    if (!m || !X || !Y) return fail(PSML_ERR_INVALID, "null argument");
-    PSML_TRY(check_ptrs({X[0], X[1], Y[0], Y[1]}));
-    m->cap_party = -1;
-    m->cap_xport = nullptr;
-    m->cap_dp = nullptr;
-    return capture_common(m, X, Y, flags, stream);
-}
-
-psml_status psml_party_capture_step(psml_model m, int32_t party, psml_xport x, psml_dp dp, const void *X_i,
-                                    const void *Y_i, int32_t flags, psml_stream stream) {
-    PSML_CTX_OPTS(m ? m->ctx : nullptr);
-    if (!m || !x) return fail(PSML_ERR_INVALID, "null model or transport");
-    if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
-    PSML_TRY(check_ptrs({X_i, Y_i}));
-    if (dp) PSML_TRY(dp_group(m, dp).st);
-    const void *X[2] = {nullptr, nullptr}, *Y[2] = {nullptr, nullptr};
-    X[party] = X_i;
-    Y[party] = Y_i;
-    m->cap_party = party;
-    m->cap_xport = x;
-    m->cap_dp = dp;
-    const psml_status st = capture_common(m, X, Y, flags, stream);
-    if (st != PSML_OK) m->cap_party = -1;
-    return st;
-}
-
 // Client encode + share of a whole minibatch in one launch (psml_model_step_host, Z_2^64): ChaCha20
 // blocks [0, nx/8) share X from 8-bit pixels (x = q / 255), the rest share Y from class indices
 // (one-hot) or float64 labels -- the same words as psml_encode_share_u8 / _onehot / encode_share.
@@ -2153,11 +2025,197 @@ __global__ void __launch_bounds__(128) client_share_kernel(const ClientJob j) {
 }
 
 // out[0..n) = a, out[n..2n) = b (the prediction shares into mapped host memory)
+static int64_t x_row(const psml_model_s *m);
+
+// The client's encode + share of the step's batch as the captured graph's first online node
+// (co-resident Z_2^64 steps): psml_model_step_device / _host point it at the batch with
+// cudaGraphExecKernelNodeSetParams before the replay (no separate launch, no launch gap between
+// it and the graph); any other replay sets it to a no-op job (nx = ny = 0).
+static ClientJob share_noop(const psml_model_s *m) {
+    ClientJob cj{};
+    cj.x0 = (T *)m->cap_X[0]; cj.x1 = (T *)m->cap_X[1]; cj.y0 = (T *)m->cap_Y[0]; cj.y1 = (T *)m->cap_Y[1];
+    return cj;
+}
+static psml_status set_share(psml_model_s *m, int g, const ClientJob &cj) {
+    cudaKernelNodeParams kp{};
+    void *args[1] = {(void *)&cj};
+    kp.func = (void *)client_share_kernel;
+    kp.gridDim = dim3(m->share_grid);
+    kp.blockDim = dim3(128);
+    kp.sharedMemBytes = 0;
+    kp.kernelParams = args;
+    PSML_CUDA_TRY(cudaGraphExecKernelNodeSetParams(m->graph[g], m->share_node[g], &kp));
+    return PSML_OK;
+}
+
+static psml_status capture_one(psml_model_s *m, int pool, const T *const X[2], const T *const Y[2], int flags,
+                               cudaStream_t s, cudaGraphExec_t *out, int64_t *kernels, int gi) {
+    const bool pipelined = (flags & 4) != 0;
+    const bool prio = pipelined && use_prio();
+    PSML_CUDA_TRY(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
+    psml_status st = PSML_OK;
+    cudaStream_t on = s;   // stream of the online phase
+    if (pipelined) {
+        if (cudaEventRecord(m->ev_fork, s) != cudaSuccess || cudaStreamWaitEvent(m->side, m->ev_fork, 0) != cudaSuccess)
+            st = fail(PSML_ERR_CUDA, "graph fork failed");
+        if (st == PSML_OK && prio) {
+            if (cudaStreamWaitEvent(m->hi, m->ev_fork, 0) != cudaSuccess) st = fail(PSML_ERR_CUDA, "graph fork failed");
+            on = m->hi;
+        }
+        const int after = cur_opts().deal_after;   // default 1: after the step-start open
+        // models without the fused step (the CNN) run large kernels that fill the GPU: their
+        // dealer forks at the start of the step (measured: 51.6K vs 49.4K samples/s forked after)
+        m->deal_after = (fused_eligible(m) && m->cap_party < 0) ? after : 0;
+        m->deal_stage = 0;
+        m->deal_on_launch = m->deal_after > 0 && cur_opts().deal_on_launch != 0;
+        if (m->deal_on_launch) m->deal_after = 2;   // the fork point right after the first product
+        m->fork_event_armed = false;
+        if (st == PSML_OK && m->deal_after == 0) {
+            st = deal_pool(m, 1 - pool, 0, false, m->side, deal_s2(m));
+            if (st == PSML_OK) advance_word_kernel<<<1, 1, 0, m->side>>>(m->step_dev);
+            if (st == PSML_OK && cudaEventRecord(m->ev_join, m->side) != cudaSuccess)
+                st = fail(PSML_ERR_CUDA, "graph join record failed");
+        } else {
+            m->deal_pending_pool = 1 - pool;   // forked from the online chain (deal_fork_point)
+        }
+    } else if (flags & 1) {
+        st = deal_pool(m, pool, 0, false, s);
+    }
+    m->pool = pool;
+    const int pp = m->cap_party;
+    const bool share_node = pp < 0 && m->ctx->ring.l == 64;
+    if (st == PSML_OK && share_node) {   // placeholder of the client's share (a no-op until set)
+        const int64_t nx = m->B * x_row(m), ny = m->B * m->dims.back();
+        m->share_grid = (unsigned)grid_for((nx + 7) / 8 + (ny + 7) / 8, 128);
+        ClientJob cj{};
+        cj.x0 = (T *)X[0]; cj.x1 = (T *)X[1]; cj.y0 = (T *)Y[0]; cj.y1 = (T *)Y[1];
+        client_share_kernel<<<m->share_grid, 128, 0, on>>>(cj);
+        if (cudaGetLastError() != cudaSuccess) st = fail(PSML_ERR_CUDA, "share node capture failed");
+    }
+    if (st == PSML_OK) {
+        if (pp >= 0) {
+            PartyRun r{m, pp, m->cap_xport, on};
+            st = party_forward_backward(r, X[pp], Y[pp]);
+        } else {
+            st = forward_backward(m, X, Y, on);
+        }
+    }
+    if (st == PSML_OK) st = deal_fork_point(m, on, true);   // not forked yet: fork here
+    m->deal_pending_pool = -1;
+    if (st == PSML_OK && (flags & 2)) {
+        m->grads_ready = true;
+        st = pp >= 0 ? party_reduce_update(m, pp, m->cap_dp, on) : psml_train_apply_update(m, 0, (psml_stream)on);
+    }
+    if (prio && st == PSML_OK &&
+        (cudaEventRecord(m->ev_hi, m->hi) != cudaSuccess || cudaStreamWaitEvent(s, m->ev_hi, 0) != cudaSuccess))
+        st = fail(PSML_ERR_CUDA, "graph join failed");
+    if (pipelined && st == PSML_OK && cudaStreamWaitEvent(s, m->ev_join, 0) != cudaSuccess)
+        st = fail(PSML_ERR_CUDA, "graph join failed");
+    cudaGraph_t g = nullptr;
+    cudaError_t e = cudaStreamEndCapture(s, &g);
+    if (st != PSML_OK) {
+        if (g) cudaGraphDestroy(g);
+        return st;
+    }
+    if (e != cudaSuccess) return fail(PSML_ERR_CUDA, std::string("graph capture: ") + cudaGetErrorString(e));
+    size_t nn = 0;
+    cudaGraphGetNodes(g, nullptr, &nn);
+    std::vector<cudaGraphNode_t> nodes(nn);
+    if (nn) cudaGraphGetNodes(g, nodes.data(), &nn);
+    *kernels = 0;
+    m->share_node[gi] = nullptr;
+    for (auto nd : nodes) {
+        cudaGraphNodeType t;
+        if (cudaGraphNodeGetType(nd, &t) == cudaSuccess && t == cudaGraphNodeTypeKernel) {
+            ++*kernels;
+            cudaKernelNodeParams kp{};
+            if (share_node && cudaGraphKernelNodeGetParams(nd, &kp) == cudaSuccess && kp.func == (void *)client_share_kernel)
+                m->share_node[gi] = nd;
+        }
+    }
+    cudaGetLastError();
+    // kernel nodes keep the priority of the stream they were captured on
+    e = cudaGraphInstantiateWithFlags(out, g, cudaGraphInstantiateFlagUseNodePriority);
+    if (e != cudaSuccess) {
+        cudaGraphDestroy(g);
+        m->share_node[gi] = nullptr;
+        return fail(PSML_ERR_CUDA, std::string("graph instantiate: ") + cudaGetErrorString(e));
+    }
+    m->graph_tmpl[gi] = g;   // kept: the share node's handle refers to it
+    m->share_live[gi] = false;
+    return PSML_OK;
+}
+
+static psml_status capture_common(psml_model m, const void *const X[2], const void *const Y[2], int32_t flags,
+                                  psml_stream stream) {
+    if (flags & ~15) return fail(PSML_ERR_INVALID, "flags: bit 0 dealer, bit 1 update, bit 2 pipelined dealer, bit 3 reuse");
+    if ((flags & 8) && (flags & 5)) return fail(PSML_ERR_INVALID, "flag bit 3 (material reuse) only applies without a dealer");
+    cudaStream_t s = (cudaStream_t)stream;
+    if (s == nullptr) return fail(PSML_ERR_INVALID, "capture needs a non-default stream");
+    for (int g = 0; g < 2; ++g) {
+        if (m->graph[g]) {
+            cudaGraphExecDestroy(m->graph[g]);
+            m->graph[g] = nullptr;
+        }
+        if (m->graph_tmpl[g]) {
+            cudaGraphDestroy(m->graph_tmpl[g]);
+            m->graph_tmpl[g] = nullptr;
+        }
+        m->share_node[g] = nullptr;
+    }
+    const int prof = g_prof_cls.exchange(-1);   // no profiling events inside the graphs
+    m->word_next = -1;
+    psml_status st = PSML_OK;
+    // one graph per dealer pool, except when the graph deals its own pool 0 (flags bit 0 only)
+    // or replays one pool on purpose (bit 3, benchmark-only material reuse)
+    const bool per_pool = (flags & 4) || !(flags & 9);
+    const int ngraphs = per_pool ? 2 : 1;
+    for (int g = 0; g < ngraphs && st == PSML_OK; ++g)
+        st = capture_one(m, per_pool ? g : 0, (const T *const *)X, (const T *const *)Y, flags, s, &m->graph[g],
+                         &m->graph_kernels, g);
+    g_prof_cls.store(prof);
+    if (st != PSML_OK) return st;
+    m->graph_flags = flags;
+    for (int i = 0; i < 2; ++i) { m->cap_X[i] = X[i]; m->cap_Y[i] = Y[i]; }
+    return PSML_OK;
+}
+
+psml_status psml_model_capture_step(psml_model m, const void *const X[2], const void *const Y[2], int32_t flags,
+                                   psml_stream stream) {
+    PSML_CTX_OPTS(m ? m->ctx : nullptr);
+    if (!m || !X || !Y) return fail(PSML_ERR_INVALID, "null argument");
+    PSML_TRY(check_ptrs({X[0], X[1], Y[0], Y[1]}));
+    m->cap_party = -1;
+    m->cap_xport = nullptr;
+    m->cap_dp = nullptr;
+    return capture_common(m, X, Y, flags, stream);
+}
+
+psml_status psml_party_capture_step(psml_model m, int32_t party, psml_xport x, psml_dp dp, const void *X_i,
+                                    const void *Y_i, int32_t flags, psml_stream stream) {
+    PSML_CTX_OPTS(m ? m->ctx : nullptr);
+    if (!m || !x) return fail(PSML_ERR_INVALID, "null model or transport");
+    if (party != 0 && party != 1) return fail(PSML_ERR_INVALID, "party must be 0 or 1");
+    PSML_TRY(check_ptrs({X_i, Y_i}));
+    if (dp) PSML_TRY(dp_group(m, dp).st);
+    const void *X[2] = {nullptr, nullptr}, *Y[2] = {nullptr, nullptr};
+    X[party] = X_i;
+    Y[party] = Y_i;
+    m->cap_party = party;
+    m->cap_xport = x;
+    m->cap_dp = dp;
+    const psml_status st = capture_common(m, X, Y, flags, stream);
+    if (st != PSML_OK) m->cap_party = -1;
+    return st;
+}
+
 template <typename U>
 __global__ void copy_pair_kernel(const U *__restrict__ a, const U *__restrict__ b, int64_t n, U *__restrict__ out) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < 2 * n; i += (int64_t)gridDim.x * blockDim.x)
         out[i] = i < n ? a[i] : b[i - n];
 }
+
+static psml_status step_graph_job(psml_model_s *m, uint32_t step_id, cudaStream_t s, const ClientJob *job);
 
 psml_status psml_model_step_host(psml_model m, const uint8_t *q, const void *y, int32_t y_kind, uint64_t share_seed,
                                  uint32_t step_id, void *yhat_host, psml_stream stream) {
@@ -2196,6 +2254,7 @@ psml_status psml_model_step_host(psml_model m, const uint8_t *q, const void *y, 
         yd = m->stage_y;
     }
     const psml_ring ring = m->ctx->ring;
+    bool shared_in_graph = false;
     const uint64_t cx = call_id(m->d.pair_id, step_id, 0, OP_SHARE, 0), cy = call_id(m->d.pair_id, step_id, 0, OP_SHARE, 1);
     if (ring.l == 64 && nx > 0 && ny > 0) {
         // X and Y in one launch: one PCIe round trip for the mapped host reads instead of two
@@ -2207,9 +2266,14 @@ psml_status psml_model_step_host(psml_model m, const uint8_t *q, const void *y, 
         cj.yf = y_kind ? nullptr : (const double *)yd;
         cj.ny = ny; cj.classes = dl;
         cj.x0 = (T *)m->cap_X[0]; cj.x1 = (T *)m->cap_X[1]; cj.y0 = (T *)m->cap_Y[0]; cj.y1 = (T *)m->cap_Y[1];
-        const int64_t blocks = (nx + 7) / 8 + (ny + 7) / 8;
-        client_share_kernel<<<grid_for(blocks, 128), 128, 0, s>>>(cj);
-        PSML_LAUNCH_CHECK();
+        if (m->share_node[0]) {   // the graph's own share node: one replay for the whole server side
+            PSML_TRY(step_graph_job(m, step_id, s, &cj));
+            shared_in_graph = true;
+        } else {
+            const int64_t blocks = (nx + 7) / 8 + (ny + 7) / 8;
+            client_share_kernel<<<grid_for(blocks, 128), 128, 0, s>>>(cj);
+            PSML_LAUNCH_CHECK();
+        }
     } else {
         PSML_TRY(psml_encode_share_u8(ring, share_seed, cx, qd, nx, 255.0, (void *)m->cap_X[0], (void *)m->cap_X[1],
                                       stream));
@@ -2221,7 +2285,7 @@ psml_status psml_model_step_host(psml_model m, const uint8_t *q, const void *y, 
                                        (void *)m->cap_Y[1], stream));
     }
     // servers: the captured step
-    PSML_TRY(psml_model_step_graph(m, step_id, stream));
+    if (!shared_in_graph) PSML_TRY(psml_model_step_graph(m, step_id, stream));
     // client: both parties' prediction shares back
     if (od) {
         copy_pair_kernel<T><<<grid_for(2 * ny, 256), 256, 0, s>>>(m->yhat.p[0], m->yhat.p[1], ny, od);
@@ -2257,6 +2321,7 @@ psml_status psml_model_step_device(psml_model m, const double *X, const double *
     cj.xf = X; cj.nx = nx; cj.f = m->ctx->ring.frac_bits;
     cj.yf = Y; cj.ny = ny; cj.classes = m->dims.back();
     cj.x0 = (T *)m->cap_X[0]; cj.x1 = (T *)m->cap_X[1]; cj.y0 = (T *)m->cap_Y[0]; cj.y1 = (T *)m->cap_Y[1];
+    if (m->share_node[0]) return step_graph_job(m, step_id, s, &cj);   // the graph's own share node
     client_share_kernel<<<grid_for((nx + 7) / 8 + (ny + 7) / 8, 128), 128, 0, s>>>(cj);
     PSML_LAUNCH_CHECK();
     return psml_model_step_graph(m, step_id, stream);
@@ -2269,11 +2334,9 @@ psml_status psml_model_graph_nodes(psml_model m, int64_t *n) {
     return PSML_OK;
 }
 
-psml_status psml_model_step_graph(psml_model m, uint32_t step_id, psml_stream stream) {
-    PSML_CTX_OPTS(m ? m->ctx : nullptr);
-    if (!m) return fail(PSML_ERR_INVALID, "model is null");
-    if (!m->graph[0]) return fail(PSML_ERR_STATE, "no captured step: call psml_model_capture_step first");
-    cudaStream_t s = (cudaStream_t)stream;
+// One replay of the captured step; job = the client's share of this step's batch for the graph's
+// share node (nullptr: the node runs as a no-op).
+static psml_status step_graph_job(psml_model_s *m, uint32_t step_id, cudaStream_t s, const ClientJob *job) {
     const bool pipelined = (m->graph_flags & 4) != 0;
     const bool self_dealt = !pipelined && (m->graph_flags & 1);
     const bool reuse = (m->graph_flags & 8) != 0;   // benchmark-only: replays pool 0 as dealt
@@ -2291,7 +2354,19 @@ psml_status psml_model_step_graph(psml_model m, uint32_t step_id, psml_stream st
         set_word_kernel<<<1, 1, 0, s>>>(m->step_dev, word);
         PSML_LAUNCH_CHECK();
     }
-    PSML_CUDA_TRY(cudaGraphLaunch(m->graph[(self_dealt || reuse) ? 0 : pool], s));
+    const int gi = (self_dealt || reuse) ? 0 : pool;
+    if (m->share_node[gi]) {
+        if (job) {
+            PSML_TRY(set_share(m, gi, *job));
+            m->share_live[gi] = true;
+        } else if (m->share_live[gi]) {
+            PSML_TRY(set_share(m, gi, share_noop(m)));
+            m->share_live[gi] = false;
+        }
+    } else if (job) {
+        return fail(PSML_ERR_STATE, "captured step has no share node");
+    }
+    PSML_CUDA_TRY(cudaGraphLaunch(m->graph[gi], s));
     m->word_next = pipelined ? (int64_t)word + 1 : -1;
     g_launches.fetch_add((uint64_t)m->graph_kernels);   // the graph's kernels are our launches
     if (pipelined) {
@@ -2305,6 +2380,13 @@ psml_status psml_model_step_graph(psml_model m, uint32_t step_id, psml_stream st
     }
     m->grads_ready = !(m->graph_flags & 2);
     return PSML_OK;
+}
+
+psml_status psml_model_step_graph(psml_model m, uint32_t step_id, psml_stream stream) {
+    PSML_CTX_OPTS(m ? m->ctx : nullptr);
+    if (!m) return fail(PSML_ERR_INVALID, "model is null");
+    if (!m->graph[0]) return fail(PSML_ERR_STATE, "no captured step: call psml_model_capture_step first");
+    return step_graph_job(m, step_id, (cudaStream_t)stream, nullptr);
 }
 
 psml_status psml_secure_infer(psml_model m, const void *const X[2], uint32_t step_id, void *const Yhat[2],
