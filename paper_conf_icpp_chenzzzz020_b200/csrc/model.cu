@@ -123,6 +123,13 @@ struct psml_model_s {
     cudaGraph_t graph_tmpl[2] = {nullptr, nullptr};  // their templates (the share node's handle lives there)
     cudaGraphNode_t share_node[2] = {nullptr, nullptr};   // the client's encode + share, first online node
     bool share_live[2] = {false, false};              // the node holds a real batch's job (else a no-op)
+    // the client's read-back of both prediction shares (psml_model_step_host into mapped pinned
+    // memory) as a graph node on its own branch, forked as soon as the forward pass wrote them
+    cudaGraphNode_t out_node[2] = {nullptr, nullptr};
+    bool out_live[2] = {false, false};
+    bool cap_out = false;              // (capture) fork the read-back branch after the forward pass
+    cudaStream_t d2h = nullptr;
+    cudaEvent_t ev_y = nullptr, ev_yj = nullptr;
     unsigned share_grid = 0;
     int graph_flags = 0;
     int64_t graph_kernels = 0;
@@ -1012,6 +1019,14 @@ static psml_status deal_fork_point(psml_model_s *m, cudaStream_t s, bool force =
 
 static bool gradw_branch() { return cur_opts().gradw_branch != 0; }
 
+// both parties' shares [a | b] (n words each) to out: the client's read-back of the predictions
+template <typename U>
+__global__ void copy_pair_kernel(const U *__restrict__ a, const U *__restrict__ b, int64_t n, U *__restrict__ out) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < 2 * n; i += (int64_t)gridDim.x * blockDim.x)
+        out[i] = i < n ? a[i] : b[i - n];
+}
+constexpr int OUT_GRID = 8;   // grid of the read-back node (2 B d_L words: a few KB)
+
 static psml_status fused_forward_backward(psml_model_s *m, const T *const X[2], const T *const Y[2], cudaStream_t s) {
     const int F = m->ctx->ring.frac_bits;
     const int nl = m->nl;
@@ -1133,6 +1148,13 @@ static psml_status fused_forward_backward(psml_model_s *m, const T *const X[2], 
                 PSML_LAUNCH_CHECK();
             }
         }
+    }
+    if (m->cap_out) {   // the read-back branch (a no-op until psml_model_step_host sets it)
+        PSML_CUDA_TRY(cudaEventRecord(m->ev_y, s));
+        PSML_CUDA_TRY(cudaStreamWaitEvent(m->d2h, m->ev_y, 0));
+        copy_pair_kernel<T><<<OUT_GRID, 256, 0, m->d2h>>>(yo[0], yo[1], 0, nullptr);
+        PSML_LAUNCH_CHECK();
+        PSML_CUDA_TRY(cudaEventRecord(m->ev_yj, m->d2h));
     }
     // 3. backward: gradW_l and gradin_l in one launch, then the backprop Hadamard opens delta_{l-1}
     //    With PSML_GRADW_BRANCH (default on), gradW_l for l > 0 runs on a second stream as soon as
@@ -1710,6 +1732,7 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
         PSML_CUDA_TRY(cudaStreamCreateWithPriority(&m->side2, cudaStreamNonBlocking, lo));
         PSML_CUDA_TRY(cudaStreamCreateWithPriority(&m->hi, cudaStreamNonBlocking, hi));
         PSML_CUDA_TRY(cudaStreamCreateWithPriority(&m->gw, cudaStreamNonBlocking, hi));
+        PSML_CUDA_TRY(cudaStreamCreateWithPriority(&m->d2h, cudaStreamNonBlocking, hi));
         PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_hi, cudaEventDisableTiming));
     }
     PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_fork, cudaEventDisableTiming));
@@ -1719,6 +1742,8 @@ psml_status psml_model_create(psml_ctx ctx, const psml_model_desc *desc, psml_mo
     PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_gw, cudaEventDisableTiming));
     PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_gwj, cudaEventDisableTiming));
     PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_d2j, cudaEventDisableTiming));
+    PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_y, cudaEventDisableTiming));
+    PSML_CUDA_TRY(cudaEventCreateWithFlags(&m->ev_yj, cudaEventDisableTiming));
     {
         T *sd = nullptr;
         PSML_TRY(dalloc(mp, &sd, 1));
@@ -1750,6 +1775,9 @@ psml_status psml_model_destroy(psml_model model) {
     if (model->gw) cudaStreamDestroy(model->gw);
     if (model->ev_gw) cudaEventDestroy(model->ev_gw);
     if (model->ev_gwj) cudaEventDestroy(model->ev_gwj);
+    if (model->ev_y) cudaEventDestroy(model->ev_y);
+    if (model->ev_yj) cudaEventDestroy(model->ev_yj);
+    if (model->d2h) cudaStreamDestroy(model->d2h);
     for (void *p : model->allocs) cudaFree(p);
     delete model;
     return PSML_OK;
@@ -2048,6 +2076,20 @@ static psml_status set_share(psml_model_s *m, int g, const ClientJob &cj) {
     return PSML_OK;
 }
 
+// the read-back node: both parties' prediction shares (n words each) to out, or a no-op (n = 0)
+static psml_status set_out(psml_model_s *m, int g, T *out, int64_t n) {
+    cudaKernelNodeParams kp{};
+    const T *a = m->yhat.p[0], *b = m->yhat.p[1];
+    void *args[4] = {(void *)&a, (void *)&b, (void *)&n, (void *)&out};
+    kp.func = (void *)copy_pair_kernel<T>;
+    kp.gridDim = dim3(OUT_GRID);
+    kp.blockDim = dim3(256);
+    kp.sharedMemBytes = 0;
+    kp.kernelParams = args;
+    PSML_CUDA_TRY(cudaGraphExecKernelNodeSetParams(m->graph[g], m->out_node[g], &kp));
+    return PSML_OK;
+}
+
 static psml_status capture_one(psml_model_s *m, int pool, const T *const X[2], const T *const Y[2], int flags,
                                cudaStream_t s, cudaGraphExec_t *out, int64_t *kernels, int gi) {
     const bool pipelined = (flags & 4) != 0;
@@ -2092,6 +2134,7 @@ static psml_status capture_one(psml_model_s *m, int pool, const T *const X[2], c
         client_share_kernel<<<m->share_grid, 128, 0, on>>>(cj);
         if (cudaGetLastError() != cudaSuccess) st = fail(PSML_ERR_CUDA, "share node capture failed");
     }
+    m->cap_out = share_node && fused_eligible(m);
     if (st == PSML_OK) {
         if (pp >= 0) {
             PartyRun r{m, pp, m->cap_xport, on};
@@ -2100,6 +2143,10 @@ static psml_status capture_one(psml_model_s *m, int pool, const T *const X[2], c
             st = forward_backward(m, X, Y, on);
         }
     }
+    if (st == PSML_OK && m->cap_out && cudaStreamWaitEvent(on, m->ev_yj, 0) != cudaSuccess)
+        st = fail(PSML_ERR_CUDA, "graph join failed");
+    const bool out_node = m->cap_out;
+    m->cap_out = false;
     if (st == PSML_OK) st = deal_fork_point(m, on, true);   // not forked yet: fork here
     m->deal_pending_pool = -1;
     if (st == PSML_OK && (flags & 2)) {
@@ -2124,13 +2171,16 @@ static psml_status capture_one(psml_model_s *m, int pool, const T *const X[2], c
     if (nn) cudaGraphGetNodes(g, nodes.data(), &nn);
     *kernels = 0;
     m->share_node[gi] = nullptr;
+    m->out_node[gi] = nullptr;
     for (auto nd : nodes) {
         cudaGraphNodeType t;
         if (cudaGraphNodeGetType(nd, &t) == cudaSuccess && t == cudaGraphNodeTypeKernel) {
             ++*kernels;
             cudaKernelNodeParams kp{};
-            if (share_node && cudaGraphKernelNodeGetParams(nd, &kp) == cudaSuccess && kp.func == (void *)client_share_kernel)
-                m->share_node[gi] = nd;
+            if ((share_node || out_node) && cudaGraphKernelNodeGetParams(nd, &kp) == cudaSuccess) {
+                if (kp.func == (void *)client_share_kernel) m->share_node[gi] = nd;
+                if (out_node && kp.func == (void *)copy_pair_kernel<T>) m->out_node[gi] = nd;
+            }
         }
     }
     cudaGetLastError();
@@ -2139,10 +2189,12 @@ static psml_status capture_one(psml_model_s *m, int pool, const T *const X[2], c
     if (e != cudaSuccess) {
         cudaGraphDestroy(g);
         m->share_node[gi] = nullptr;
+        m->out_node[gi] = nullptr;
         return fail(PSML_ERR_CUDA, std::string("graph instantiate: ") + cudaGetErrorString(e));
     }
     m->graph_tmpl[gi] = g;   // kept: the share node's handle refers to it
     m->share_live[gi] = false;
+    m->out_live[gi] = false;
     return PSML_OK;
 }
 
@@ -2162,6 +2214,7 @@ static psml_status capture_common(psml_model m, const void *const X[2], const vo
             m->graph_tmpl[g] = nullptr;
         }
         m->share_node[g] = nullptr;
+        m->out_node[g] = nullptr;
     }
     const int prof = g_prof_cls.exchange(-1);   // no profiling events inside the graphs
     m->word_next = -1;
@@ -2209,13 +2262,9 @@ psml_status psml_party_capture_step(psml_model m, int32_t party, psml_xport x, p
     return st;
 }
 
-template <typename U>
-__global__ void copy_pair_kernel(const U *__restrict__ a, const U *__restrict__ b, int64_t n, U *__restrict__ out) {
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < 2 * n; i += (int64_t)gridDim.x * blockDim.x)
-        out[i] = i < n ? a[i] : b[i - n];
-}
 
-static psml_status step_graph_job(psml_model_s *m, uint32_t step_id, cudaStream_t s, const ClientJob *job);
+static psml_status step_graph_job(psml_model_s *m, uint32_t step_id, cudaStream_t s, const ClientJob *job,
+                                  T *out, int64_t out_n);
 
 psml_status psml_model_step_host(psml_model m, const uint8_t *q, const void *y, int32_t y_kind, uint64_t share_seed,
                                  uint32_t step_id, void *yhat_host, psml_stream stream) {
@@ -2254,7 +2303,7 @@ psml_status psml_model_step_host(psml_model m, const uint8_t *q, const void *y, 
         yd = m->stage_y;
     }
     const psml_ring ring = m->ctx->ring;
-    bool shared_in_graph = false;
+    bool shared_in_graph = false, read_in_graph = false;
     const uint64_t cx = call_id(m->d.pair_id, step_id, 0, OP_SHARE, 0), cy = call_id(m->d.pair_id, step_id, 0, OP_SHARE, 1);
     if (ring.l == 64 && nx > 0 && ny > 0) {
         // X and Y in one launch: one PCIe round trip for the mapped host reads instead of two
@@ -2267,7 +2316,8 @@ psml_status psml_model_step_host(psml_model m, const uint8_t *q, const void *y, 
         cj.ny = ny; cj.classes = dl;
         cj.x0 = (T *)m->cap_X[0]; cj.x1 = (T *)m->cap_X[1]; cj.y0 = (T *)m->cap_Y[0]; cj.y1 = (T *)m->cap_Y[1];
         if (m->share_node[0]) {   // the graph's own share node: one replay for the whole server side
-            PSML_TRY(step_graph_job(m, step_id, s, &cj));
+            read_in_graph = od && m->out_node[0];   // ... and its read-back node, beside the backward pass
+            PSML_TRY(step_graph_job(m, step_id, s, &cj, read_in_graph ? od : nullptr, ny));
             shared_in_graph = true;
         } else {
             const int64_t blocks = (nx + 7) / 8 + (ny + 7) / 8;
@@ -2287,7 +2337,9 @@ psml_status psml_model_step_host(psml_model m, const uint8_t *q, const void *y, 
     // servers: the captured step
     if (!shared_in_graph) PSML_TRY(psml_model_step_graph(m, step_id, stream));
     // client: both parties' prediction shares back
-    if (od) {
+    if (read_in_graph) {
+        // done by the graph's read-back node
+    } else if (od) {
         copy_pair_kernel<T><<<grid_for(2 * ny, 256), 256, 0, s>>>(m->yhat.p[0], m->yhat.p[1], ny, od);
         PSML_LAUNCH_CHECK();
     } else {
@@ -2321,7 +2373,7 @@ psml_status psml_model_step_device(psml_model m, const double *X, const double *
     cj.xf = X; cj.nx = nx; cj.f = m->ctx->ring.frac_bits;
     cj.yf = Y; cj.ny = ny; cj.classes = m->dims.back();
     cj.x0 = (T *)m->cap_X[0]; cj.x1 = (T *)m->cap_X[1]; cj.y0 = (T *)m->cap_Y[0]; cj.y1 = (T *)m->cap_Y[1];
-    if (m->share_node[0]) return step_graph_job(m, step_id, s, &cj);   // the graph's own share node
+    if (m->share_node[0]) return step_graph_job(m, step_id, s, &cj, nullptr, 0);   // the graph's own share node
     client_share_kernel<<<grid_for((nx + 7) / 8 + (ny + 7) / 8, 128), 128, 0, s>>>(cj);
     PSML_LAUNCH_CHECK();
     return psml_model_step_graph(m, step_id, stream);
@@ -2336,7 +2388,8 @@ psml_status psml_model_graph_nodes(psml_model m, int64_t *n) {
 
 // One replay of the captured step; job = the client's share of this step's batch for the graph's
 // share node (nullptr: the node runs as a no-op).
-static psml_status step_graph_job(psml_model_s *m, uint32_t step_id, cudaStream_t s, const ClientJob *job) {
+static psml_status step_graph_job(psml_model_s *m, uint32_t step_id, cudaStream_t s, const ClientJob *job,
+                                  T *out = nullptr, int64_t out_n = 0) {
     const bool pipelined = (m->graph_flags & 4) != 0;
     const bool self_dealt = !pipelined && (m->graph_flags & 1);
     const bool reuse = (m->graph_flags & 8) != 0;   // benchmark-only: replays pool 0 as dealt
@@ -2366,6 +2419,17 @@ static psml_status step_graph_job(psml_model_s *m, uint32_t step_id, cudaStream_
     } else if (job) {
         return fail(PSML_ERR_STATE, "captured step has no share node");
     }
+    if (m->out_node[gi]) {
+        if (out) {
+            PSML_TRY(set_out(m, gi, out, out_n));
+            m->out_live[gi] = true;
+        } else if (m->out_live[gi]) {
+            PSML_TRY(set_out(m, gi, nullptr, 0));
+            m->out_live[gi] = false;
+        }
+    } else if (out) {
+        return fail(PSML_ERR_STATE, "captured step has no read-back node");
+    }
     PSML_CUDA_TRY(cudaGraphLaunch(m->graph[gi], s));
     m->word_next = pipelined ? (int64_t)word + 1 : -1;
     g_launches.fetch_add((uint64_t)m->graph_kernels);   // the graph's kernels are our launches
@@ -2386,7 +2450,7 @@ psml_status psml_model_step_graph(psml_model m, uint32_t step_id, psml_stream st
     PSML_CTX_OPTS(m ? m->ctx : nullptr);
     if (!m) return fail(PSML_ERR_INVALID, "model is null");
     if (!m->graph[0]) return fail(PSML_ERR_STATE, "no captured step: call psml_model_capture_step first");
-    return step_graph_job(m, step_id, (cudaStream_t)stream, nullptr);
+    return step_graph_job(m, step_id, (cudaStream_t)stream, nullptr, nullptr, 0);
 }
 
 psml_status psml_secure_infer(psml_model m, const void *const X[2], uint32_t step_id, void *const Yhat[2],
