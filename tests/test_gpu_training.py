@@ -146,6 +146,44 @@ def test_step_host_bitexact_vs_oracle(T, task):
     tr.close()
 
 
+def test_graph_share_and_readback_nodes_switch_between_entry_points(T):
+    """The captured graph's client-share and read-back nodes are parameterised per replay:
+    psml_model_step_host points them at its pinned buffers, psml_model_step_device sets only the
+    share node, and a plain replay (host-side share into the captured buffers + psml_model_step_graph)
+    runs both as no-ops.  Interleaving the three entry points must stay bit-exact vs the oracle, and a
+    replay that is not step_host must not write into an earlier step_host's output buffer."""
+    task = "mlp"
+    Wi = synth.init_weights(task)
+    tr = T.SecureTrainer(task, Wi, backend=0)
+    om = OP.Model(task, Wi)
+    X, Y = synth.batch(task, 0)
+    tr.step(torch.from_numpy(X), torch.from_numpy(Y), 0)
+    OP.train_step(om, X, Y, 0)
+    tr.capture(pipelined=True)
+    outs = {}
+    for s, how in ((1, "host"), (2, "plain"), (3, "device"), (4, "host"), (5, "device"), (6, "plain"), (7, "host")):
+        X, Y = synth.batch(task, s)
+        if how == "host":
+            q, y = synth.batch_u8(task, s)
+            out = torch.zeros((2, X.shape[0], Y.shape[1]), dtype=torch.uint64).pin_memory()
+            tr.graph_step_host(torch.from_numpy(q).pin_memory(),
+                               torch.from_numpy(np.ascontiguousarray(y)).pin_memory(), s, out)
+        elif how == "device":
+            tr.graph_step(torch.from_numpy(X).cuda(), torch.from_numpy(Y).cuda(), s)
+        else:
+            tr.graph_step(torch.from_numpy(X), torch.from_numpy(Y), s)   # host share + plain replay
+        yhat = OP.train_step(om, X, Y, s)
+        torch.cuda.synchronize()
+        _compare_shares(tr, om)
+        if how == "host":
+            for i in range(2):
+                assert np.array_equal(out[i].numpy(), yhat[i].reshape(out[i].shape)), (s, i)
+            outs[s] = (out, out.clone())
+        for k, (buf, snap) in outs.items():   # earlier step_host buffers stay untouched
+            assert torch.equal(buf, snap), (k, s, how)
+    tr.close()
+
+
 @pytest.mark.parametrize("task", ["mlp", "logreg"])
 def test_one_epoch_bench_path_bitexact_vs_eager_and_fp64(T, task):
     """The launch configuration bench.py times -- pipelined CUDA graph (dealer of step s+1 forked
