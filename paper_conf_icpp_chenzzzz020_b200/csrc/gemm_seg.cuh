@@ -249,9 +249,13 @@ bool tc_seg_enabled();
 bool tc_seg_forced();   // PSML_SEG=tc: every eligible group on tcgen05 (tests)
 bool pdl_enabled();     // PSML_PDL=0 disables programmatic dependent launch
 // segs = 2: Beaver products [X_p | E] . [F ; V_p]; 1: plain X . F.  fill: the grid's K split stops at
-// 1/fill of the SMs (2 inside the training step, whose dealer branch runs beside it; 1 stand-alone).
+// 2/fill of the SMs (2 inside the training step, whose dealer branch runs beside it; 0 stand-alone:
+// one wave of one-CTA-per-SM clusters).
+#ifndef PSML_TCSEG_FILL
+#define PSML_TCSEG_FILL 2
+#endif
 psml_status tc_seg_group(const SegArgs<uint64_t> *jobs, int njobs, cudaStream_t stream, int sm_count, int segs = 2,
-                         int fill = 2);
+                         int fill = PSML_TCSEG_FILL);
 // Stand-alone products on the in-kernel limb-split kernel (psml_options.tc_small): plain C = A . B
 // and the co-resident Beaver product (one mask + open pass, then Eq. 8); l = 64 needs K' <= 16384.
 bool tc_seg_small(int l, int64_t M, int64_t Kext, int64_t N, int nparty, int sm_count);

@@ -547,10 +547,11 @@ static psml_status tc_seg_group_t(const SegArgs<T> *jobs, int njobs, cudaStream_
     g.tile_begin[njobs] = tiles;
     g.njobs = njobs;
     g.segs = segs;
-    // K split: double ks while the grid stays within 1/fill of the SMs (training step: 2, the rest
-    // stays with the dealer branch; stand-alone products: 1) and each split keeps >= 2 K blocks
+    // K split: double ks while the grid stays within 2/fill of the SMs (training step, fill = 2: the
+    // rest stays with the dealer branch; fill = 0: stand-alone products, one wave) and each split
+    // keeps >= 2 K blocks
     int ks = 1;
-    if (fill > 1) {   // training step (measured: up to 2 sm_count / fill CTAs)
+    if (fill > 0) {   // training step (measured: up to 2 sm_count / fill CTAs)
         while (ks < max_ks && tiles * ks * 2 * fill <= 2 * sm_count && nkb_max >= ks * 2) ks *= 2;
     } else {          // stand-alone: the whole grid in one wave of one-CTA-per-SM clusters
         while (ks < max_ks && tiles * ks * 2 <= sm_count && nkb_max >= ks * 2) ks *= 2;
@@ -611,7 +612,7 @@ psml_status tc_seg_plain(const T *A, const T *B, int64_t M, int64_t K, int64_t N
     SegArgs<T> a{};
     a.X[0] = A; a.F = B; a.C[0] = C;
     a.M = M; a.N = N; a.K = K; a.trunc = 0; a.nparty = 1;
-    return tc_seg_group_t<T>(&a, 1, s, sm_count, 1, 1);
+    return tc_seg_group_t<T>(&a, 1, s, sm_count, 1, 0);
 }
 
 template <typename T>
@@ -643,7 +644,7 @@ psml_status tc_seg_beaver(const T *const A[2], const T *const B[2], const T *con
     a.X[0] = U[0]; a.X[1] = X1; a.E = E; a.F = F;
     for (int p = 0; p < 2; ++p) { a.V[p] = V[p]; a.Z[p] = Z[p]; a.C[p] = C[p]; a.party[p] = p; }
     a.M = M; a.N = N; a.K = K; a.trunc = trunc; a.nparty = 2;
-    return tc_seg_group_t<T>(&a, 1, s, sm_count, 2, 1);
+    return tc_seg_group_t<T>(&a, 1, s, sm_count, 2, 0);
 }
 
 #define PSML_TCSEG_INST(T)                                                                                        \
