@@ -530,7 +530,8 @@ def committed_traffic(name):
     for f in sorted(glob.glob(os.path.join(ROOT, "profiles", "r0*_traffic.json")), reverse=True):
         try:
             t = json.load(open(f))
-            return t[name]["bytes_per_launch_avg"], t["source"]
+            # the committed summary this value is read from (its source capture stays out of the tree)
+            return t[name]["bytes_per_launch_avg"], f"{os.path.relpath(f, ROOT)} (from {t['source']})"
         except (OSError, ValueError, KeyError):
             continue
     return None, None
