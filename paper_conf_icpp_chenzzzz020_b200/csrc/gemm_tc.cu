@@ -257,9 +257,6 @@ __device__ __forceinline__ void epi_chunk(T *st, const T v[16], int lane, int64_
     __syncwarp();
 }
 
-#ifndef TC_V1_GROUP
-#define TC_V1_GROUP 1   // BN = 128: no gain (4096^3 0.5745 vs 0.5724 ms); BN = 64: 4 MMAs of N <= 256 per block
-#endif
 #ifndef TC_B_MULTICAST
 #define TC_B_MULTICAST 1
 #endif
@@ -276,7 +273,6 @@ __global__ void __launch_bounds__(128, (STAGES * L * (BM * BK + BN * BK) <= 110 
     // share an SM, one's epilogue overlapping the other's main loop)
     constexpr uint32_t TCOLS = L * BN <= 32 ? 32 : L * BN <= 64 ? 64 : L * BN <= 128 ? 128 : L * BN <= 256 ? 256 : 512;
     constexpr int STAGE_BYTES = L * (A_BYTES + B_BYTES);
-    constexpr uint32_t IDESC = idesc_i8(BM, BN);
     uint64_t *full = (uint64_t *)(smem + STAGES * STAGE_BYTES);
     uint64_t *empty = full + STAGES;
     uint64_t *accum = empty + STAGES;
@@ -343,7 +339,6 @@ __global__ void __launch_bounds__(128, (STAGES * L * (BM * BK + BN * BK) <= 110 
             mbar_wait(smem_u32(&full[stage]), phase);
             tc_fence_after();
             const uint32_t sa = smem_u32(smem + stage * STAGE_BYTES), sb = sa + L * A_BYTES;
-#if TC_V1_GROUP
             // the B planes q0, q0 + 1 of A limb p lie back to back in the canonical layout (plane
             // stride = BN / 8 row groups x SBO): ONE N = 2 BN operand into the adjacent shift
             // accumulators S_{p+q0}, S_{p+q0+1} -- 6 MMAs per block instead of 10 at l = 32, A read
@@ -360,17 +355,6 @@ __global__ void __launch_bounds__(128, (STAGES * L * (BM * BK + BN * BK) <= 110 
                               (kb > kb0 || p > 0) ? 1u : 0u);
                 }
             }
-#else
-#pragma unroll
-            for (int p = 0; p < L; ++p) {
-                const uint64_t ad = smem_desc(sa + p * A_BYTES, 128, 256);
-#pragma unroll
-                for (int q = 0; q < L - p; ++q) {
-                    const uint64_t bd = smem_desc(sb + q * B_BYTES, 128, 256);
-                    tc_mma_i8(tmem + (uint32_t)((p + q) * BN), ad, bd, IDESC, (kb > kb0 || p > 0) ? 1u : 0u);
-                }
-            }
-#endif
             if (MC > 1) tc_commit_mc(smem_u32(&empty[stage]), (1u << MC) - 1);   // both CTAs' copies of the stage
             else tc_commit(smem_u32(&empty[stage]));   // frees the smem stage once these MMAs retire
             if (++stage == STAGES) { stage = 0; phase ^= 1; }

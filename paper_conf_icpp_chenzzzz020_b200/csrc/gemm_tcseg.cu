@@ -509,9 +509,6 @@ static psml_status tc_seg_group_t(const SegArgs<T> *jobs, int njobs, cudaStream_
     static int max_ks = 8;
     if (!attr_done) {
         PSML_CUDA_TRY(cudaFuncSetAttribute(tcseg::tc_seg_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)SMEM_BYTES));
-#ifdef TCSEG_CARVEOUT
-        PSML_CUDA_TRY(cudaFuncSetAttribute(tcseg::tc_seg_kernel<T>, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
-#endif
         if (cudaFuncSetAttribute(tcseg::tc_seg_kernel<T>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1) == cudaSuccess) {
             cudaLaunchConfig_t q = {};
             q.gridDim = dim3(MAX_KS, 1, MAX_KS);
