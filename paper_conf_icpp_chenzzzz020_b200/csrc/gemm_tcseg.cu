@@ -11,7 +11,7 @@
 // byte transpose per 4 words: 2 PRMT per limb word) and store them into shared memory in the UMMA
 // K-major no-swizzle canonical layout; warp 8 issues the block's limb-pair MMAs (the B planes of
 // one A limb as one N <= 256 operand: 12 MMAs per block) as soon as the stage's `full` barrier
-// completes (4-stage ring; the commit of a stage's MMAs frees it).  Per 128 x 64 x 32 block a CTA
+// completes (3-stage ring; the commit of a stage's MMAs frees it).  Per 128 x 64 x 32 block a CTA
 // moves 48 KB of limb planes into shared memory and the MMAs read 120 KB back (A 12 x 4 KB, B
 // 36 x 2 KB): 168 KB at 128 B/clk is 1.3 us -- the kernel's shared-memory roofline (measured
 // 1.4 us per block with every SM busy).
@@ -30,7 +30,10 @@ namespace psml {
 namespace tcseg {
 
 constexpr int BM = 128, BN = 64, BK = 32, NT = 256, LMAX = 8;
-constexpr int STAGES = 4;
+#ifndef TCSEG_STAGES
+#define TCSEG_STAGES 3   // limb-stage ring (same box: 4 -> 3 stages 1024^3 55.3 -> 53.2 us, step unchanged; 2 slower e2e)
+#endif
+constexpr int STAGES = TCSEG_STAGES;
 constexpr int NTH = NT + 32;   // NT producer threads (loads, limb split, epilogue) + the MMA warp
 constexpr int A_TILE = BM * BK;                        // bytes per limb plane of one A block
 constexpr int B_TILE = BN * BK;                        // bytes per limb plane of one B block
