@@ -125,8 +125,8 @@ typedef struct {
                               the deal_after-th online stage completes                          */
     int32_t tc_small;      /* stand-alone psml_ring_gemm / co-resident psml_secure_matmul in Z_2^64
                               (BASELINE config 5 at small n) on tcgen05: 1 auto = products whose
-                              128 x 64 output tiles (x 2 parties) fit one wave of the SMs and
-                              K' <= 16384 run on the in-kernel limb-split kernel (one launch,
+                              128 x 64 output tiles (x 2 parties) fit one wave of the SMs (two
+                              waves at l = 64) and K' <= 16384 run on the in-kernel limb-split kernel (one launch,
                               cluster split-K over the whole GPU), larger ones on the limb-plane
                               kernels; 0 always the limb-plane kernels; 2 the in-kernel split
                               kernel wherever K' <= 16384                                       */

@@ -601,10 +601,13 @@ bool tc_seg_small(int l, int64_t M, int64_t Kext, int64_t N, int nparty, int sm_
     const int mode = cur_opts().tc_small;   // psml_options.tc_small
     if (mode == 0 || !tc_seg_enabled() || (l == 64 && Kext > 16384) || M <= 0 || N <= 0) return false;
     if (mode == 2) return true;
-    // auto: the output tiles fit one wave (measured, tools/tc_small_ab.py: 512^3 plain 44 -> 20 us,
-    // 1024^3 plain 93 -> 64 us; Beaver 1024^3 (256 tiles, two waves) is faster on the limb planes)
+    // auto: the output tiles fit one wave, two for l = 64 (measured, tools/tc_small_ab.py and the
+    // config-5 sweep: 512^3 plain 44 -> 18.5 us, 1024^3 plain 93 -> 52 us; Beaver 1024^3 (256 tiles)
+    // l = 64 224 -> 204 us, but l = 32 112 us on the limb planes vs 142; 2048^3 plain l = 64 280 us on
+    // the limb planes vs 330)
     using namespace tcseg;
-    return ((M + BM - 1) / BM) * ((N + BN - 1) / BN) * nparty <= sm_count;
+    const int64_t tiles = ((M + BM - 1) / BM) * ((N + BN - 1) / BN) * nparty;
+    return tiles <= (l == 64 ? 2 : 1) * (int64_t)sm_count;
 }
 
 template <typename T>
