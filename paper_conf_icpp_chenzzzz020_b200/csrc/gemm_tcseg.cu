@@ -144,6 +144,14 @@ __device__ __forceinline__ void ld4(const uint32_t *p, uint32_t *v) {
     const uint4 q = __ldg((const uint4 *)p);
     v[0] = q.x; v[1] = q.y; v[2] = q.z; v[3] = q.w;
 }
+// one A unit of UW consecutive words in one load: 32 B (4 x u64 or 8 x u32; aligned)
+__device__ __forceinline__ void ld_unit(const uint64_t *p, uint64_t *v) { ld4(p, v); }
+__device__ __forceinline__ void ld_unit(const uint32_t *p, uint32_t *v) {
+    uint64_t a, b, c, d;
+    asm volatile("ld.global.nc.v4.u64 {%0, %1, %2, %3}, [%4];" : "=l"(a), "=l"(b), "=l"(c), "=l"(d) : "l"(p));
+    v[0] = (uint32_t)a; v[1] = (uint32_t)(a >> 32); v[2] = (uint32_t)b; v[3] = (uint32_t)(b >> 32);
+    v[4] = (uint32_t)c; v[5] = (uint32_t)(c >> 32); v[6] = (uint32_t)d; v[7] = (uint32_t)(d >> 32);
+}
 __device__ __forceinline__ uint64_t ld_dsmem(uint32_t a, uint64_t *) {
     uint64_t v;
     asm volatile("ld.shared::cluster.u64 %0, [%1];" : "=l"(v) : "r"(a));
@@ -304,16 +312,19 @@ __global__ void __launch_bounds__(NTH, 1) tc_seg_kernel(const __grid_constant__ 
         // shared memory once -- as limb planes -- instead of raw words in + out + limb planes.
         const int64_t bnn = n0 + bn;
         const bool bcol = bnn < N;
-        auto alv = [](const void *q) { return ((uintptr_t)q & (4 * sizeof(T) - 1)) == 0; };
-        const bool a32 = (K % 4) == 0 && alv(Xp) && alv(Ep);
+        // an A unit is UW consecutive k of one row = 32 bytes (4 words at l = 64, 8 at l = 32):
+        // NU units per thread, UPR units per 32-k row of the block
+        constexpr int UW = 32 / (int)sizeof(T), NU = 16 / UW, UPR = BK / UW;
+        auto alv = [](const void *q) { return ((uintptr_t)q & 31) == 0; };
+        const bool a32 = (K % UW) == 0 && alv(Xp) && alv(Ep);
         // interior blocks (every row / column inside, the 32 k inside one segment) take a fast path:
         // precomputed row offsets, no bounds checks, one address add per load
         const bool rows_full = m0 + BM <= M && a32, cols_full = n0 + BN <= N;
-        int64_t rowoff[4];
+        int64_t rowoff[NU];
 #pragma unroll
-        for (int i = 0; i < 4; ++i) {
+        for (int i = 0; i < NU; ++i) {
             const int u = tid + NT * i;
-            rowoff[i] = (m0 + (u >> 3)) * K + 4 * (u & 7);
+            rowoff[i] = (m0 + u / UPR) * K + UW * (u % UPR);
         }
         const int64_t colbase = (int64_t)(8 * bq) * N + bnn;
         auto load = [&](int kb, T (&va)[16], T (&vb)[8]) {
@@ -322,24 +333,25 @@ __global__ void __launch_bounds__(NTH, 1) tc_seg_kernel(const __grid_constant__ 
             if (rows_full && one_seg) {
                 const T *sb = k0 < K ? Xp + k0 : Ep + (k0 - K);
 #pragma unroll
-                for (int i = 0; i < 4; ++i) ld4(sb + rowoff[i], va + 4 * i);
+                for (int i = 0; i < NU; ++i) ld_unit(sb + rowoff[i], va + UW * i);
             } else {
 #pragma unroll
-                for (int i = 0; i < 4; ++i) {
-                    const int u = tid + NT * i, row = u >> 3;
-                    const int64_t m = m0 + row, k = k0 + 4 * (u & 7);
+                for (int i = 0; i < NU; ++i) {
+                    const int u = tid + NT * i, row = u / UPR;
+                    const int64_t m = m0 + row, k = k0 + UW * (u % UPR);
                     const int64_t mc = m < M ? m : 0;
                     if (a32) {
                         if (m < M && k < Kext) {
-                            ld4(k < K ? Xp + mc * K + k : Ep + mc * K + (k - K), va + 4 * i);
+                            ld_unit(k < K ? Xp + mc * K + k : Ep + mc * K + (k - K), va + UW * i);
                         } else {
-                            va[4 * i] = va[4 * i + 1] = va[4 * i + 2] = va[4 * i + 3] = 0;
+#pragma unroll
+                            for (int j = 0; j < UW; ++j) va[UW * i + j] = 0;
                         }
                     } else {
 #pragma unroll
-                        for (int j = 0; j < 4; ++j) {
+                        for (int j = 0; j < UW; ++j) {
                             const int64_t kk = k + j;
-                            va[4 * i + j] = (m < M && kk < Kext) ? ldg(kk < K ? Xp + mc * K + kk : Ep + mc * K + (kk - K)) : 0;
+                            va[UW * i + j] = (m < M && kk < Kext) ? ldg(kk < K ? Xp + mc * K + kk : Ep + mc * K + (kk - K)) : 0;
                         }
                     }
                 }
@@ -360,13 +372,22 @@ __global__ void __launch_bounds__(NTH, 1) tc_seg_kernel(const __grid_constant__ 
         auto stash_regs = [&](int st, const T (&va)[16], const T (&vb)[8]) {
             uint8_t *sa = smem + st * STAGE_BYTES, *sb = sa + L * A_TILE;
 #pragma unroll
-            for (int i = 0; i < 4; ++i) {
-                const int u = tid + NT * i, row = u >> 3, c = u & 7;
-                const int off = (((row >> 3) * 2 + (c >> 2)) * 128) + (row & 7) * 16 + (c & 3) * 4;
-                uint32_t w[L];
-                limbs4(va + 4 * i, w);
+            for (int i = 0; i < NU; ++i) {
+                const int u = tid + NT * i, row = u / UPR, k = UW * (u % UPR);
+                // the unit's k range inside the 16-byte core-matrix row of each limb plane
+                const int off = (((row >> 3) * 2 + (k >> 4)) * 128) + (row & 7) * 16 + (k & 15);
+                if constexpr (UW == 4) {
+                    uint32_t w[L];
+                    limbs4(va + UW * i, w);
 #pragma unroll
-                for (int l = 0; l < L; ++l) *(uint32_t *)(sa + l * A_TILE + off) = w[l];
+                    for (int l = 0; l < L; ++l) *(uint32_t *)(sa + l * A_TILE + off) = w[l];
+                } else {   // 8 k: two limb words per plane, one 8-byte store
+                    uint32_t w0[L], w1[L];
+                    limbs4(va + UW * i, w0);
+                    limbs4(va + UW * i + 4, w1);
+#pragma unroll
+                    for (int l = 0; l < L; ++l) *(uint2 *)(sa + l * A_TILE + off) = make_uint2(w0[l], w1[l]);
+                }
             }
             uint32_t u[2][L];
             limbs4(vb, u[0]);
